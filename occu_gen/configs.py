@@ -1,0 +1,162 @@
+"""Seeded synthetic workloads for the BASELINE.json configs.
+
+Every batch is (graphs, node_feat, edge_feat, targets):
+  graphs     list of (num_nodes, src int32[m], dst int32[m]) with local ids
+  node_feat  float32 [N, F_n]   graphs concatenated in caller order
+  edge_feat  float32 [E, F_e]   graphs concatenated, INPUT edge order
+  targets    float32 [B]        synthetic teacher labels in (0, 1)
+Seeds: generator seed 1000 + config index.
+"""
+from __future__ import annotations
+
+from dataclasses import dataclass
+
+import numpy as np
+
+from . import dags
+from .features import F_E, F_N, node_edge_features
+from .prng import Rng, uniform01
+
+
+@dataclass
+class Batch:
+    graphs: list
+    node_feat: np.ndarray
+    edge_feat: np.ndarray
+    targets: np.ndarray
+    families: list
+
+    @property
+    def num_graphs(self):
+        return len(self.graphs)
+
+    @property
+    def num_nodes(self):
+        return int(sum(g[0] for g in self.graphs))
+
+    @property
+    def num_edges(self):
+        return int(sum(len(g[1]) for g in self.graphs))
+
+    def subset(self, idx):
+        """Batch of graphs ``idx`` (in that order), features sliced accordingly."""
+        noff = np.concatenate([[0], np.cumsum([g[0] for g in self.graphs])])
+        eoff = np.concatenate([[0], np.cumsum([len(g[1]) for g in self.graphs])])
+        nf = [self.node_feat[noff[i]:noff[i + 1]] for i in idx]
+        ef = [self.edge_feat[eoff[i]:eoff[i + 1]] for i in idx]
+        return Batch([self.graphs[i] for i in idx],
+                     np.concatenate(nf) if nf else np.zeros((0, self.node_feat.shape[1]), np.float32),
+                     np.concatenate(ef) if ef else np.zeros((0, self.edge_feat.shape[1]), np.float32),
+                     self.targets[list(idx)].copy(), [self.families[i] for i in idx])
+
+
+def teacher_targets(node_feat_list, seed: int) -> np.ndarray:
+    """Synthetic labels: sigmoid of a seeded linear function of mean node features.
+
+    Stands in for profiled occupancy (P85-P95), which needs the paper's GPUs.
+    """
+    w = 2.0 * uniform01(seed, F_N) - 1.0
+    ys = []
+    for X in node_feat_list:
+        z = 4.0 * float(X.astype(np.float64).mean(axis=0) @ w)
+        ys.append(1.0 / (1.0 + np.exp(-z)))
+    return np.asarray(ys, np.float32)
+
+
+def _make(families_hp, gpu="A100", seed=0):
+    graphs, nfs, efs, fams = [], [], [], []
+    for fam, hp in families_hp:
+        g = dags.training_graph(fam, hp)
+        X, E = node_edge_features(g, dict(dags.default_hp(fam), **hp), gpu)
+        graphs.append((g.num_nodes, g.src, g.dst))
+        nfs.append(X)
+        efs.append(E)
+        fams.append(fam)
+    y = teacher_targets(nfs, seed + 7)
+    return Batch(graphs, np.concatenate(nfs), np.concatenate(efs), y, fams)
+
+
+def cnn_grid():
+    """CNN variants: batch in {16,20..128} x C_in in 1..10, lexicographic (P237)."""
+    return [{"batch": b, "cin": c} for b in range(16, 129, 4) for c in range(1, 11)]
+
+
+def cfg1():
+    """CFG1: one LeNet-5 training graph (~40 nodes); L=2, d=64, FP32 forward."""
+    return _make([("lenet5", {"batch": 16, "cin": 1})], seed=1001)
+
+
+def cfg2(num_graphs: int = 256):
+    """CFG2: ResNet-50 training graphs, first 256 variants of the batch x C_in grid."""
+    grid = cnn_grid()
+    hps = [grid[i % len(grid)] for i in range(num_graphs)]
+    return _make([("resnet50", hp) for hp in hps], seed=1002)
+
+
+def transformer_variants(n: int, seed: int):
+    r = Rng(seed)
+    out = []
+    for _ in range(n):
+        out.append({"batch": int(4 * r.randint(4, 32)[0]), "cin": int(r.randint(1, 10)[0]),
+                    "seq": int(r.choice([20, 512]))})
+    return out
+
+
+def cfg3(num_graphs: int = 512):
+    """CFG3: BERT-base / GPT-2 training graphs (~5k nodes), half each."""
+    hps = transformer_variants(num_graphs, 1003)
+    fams = ["bert_base" if i < num_graphs // 2 else "gpt2" for i in range(num_graphs)]
+    return _make(list(zip(fams, hps)), seed=1003)
+
+
+def mixture_variant(family: str, r: Rng) -> dict:
+    if family in dags.RNN:
+        return {"batch": int(8 * r.randint(16, 64)[0]), "seq": int(8 * r.randint(2, 16)[0])}
+    if family in dags.TRANSFORMER:
+        return {"batch": int(4 * r.randint(4, 32)[0]), "cin": int(r.randint(1, 10)[0]),
+                "seq": int(r.choice([20, 512]))}
+    return {"batch": int(4 * r.randint(4, 32)[0]), "cin": int(r.randint(1, 10)[0])}
+
+
+MIXTURE = [f for f in dags.FAMILIES if f != "bert_base"]   # the 20 Table II models
+
+
+def mixture(num_graphs: int, seed: int, start: int = 0):
+    """Graphs ``start .. start+num_graphs-1`` of the 20-family mixture (CFG4/CFG5)."""
+    out = []
+    for k in range(start, start + num_graphs):
+        r = Rng((seed << 32) + k)
+        fam = MIXTURE[int(r.randint(0, len(MIXTURE) - 1)[0])]
+        out.append((fam, mixture_variant(fam, r)))
+    return _make(out, seed=seed)
+
+
+def random_dag_batch(num_graphs: int, seed: int, max_nodes: int = 12, hub: bool = False,
+                     f_n: int = F_N, f_e: int = F_E, allow_empty_edges: bool = True):
+    """Small random DAGs (edges u<v, multi-edges allowed) with uniform features.
+
+    Used for fuzzing the packer and for oracle / parity tests at tiny sizes.
+    """
+    r = Rng(seed)
+    graphs, nfs, efs = [], [], []
+    for _ in range(num_graphs):
+        n = int(r.randint(1, max_nodes)[0])
+        if n == 1:
+            m = 0
+        else:
+            lo = 0 if allow_empty_edges else 1
+            m = int(r.randint(lo, 2 * n)[0])
+        s = r.randint(0, max(n - 2, 0), m) if m else np.zeros(0, np.int64)
+        span = (n - 1 - s)
+        t = s + 1 + np.floor(r.uniform(m) * span).astype(np.int64) if m else np.zeros(0, np.int64)
+        if hub and n > 2 and m:
+            h = n - 1
+            extra = int(r.randint(1, 3 * n)[0])
+            s = np.concatenate([s, r.randint(0, h - 1, extra)])
+            t = np.concatenate([t, np.full(extra, h)])
+        graphs.append((n, s.astype(np.int32), t.astype(np.int32)))
+        nfs.append(r.uniform(n * f_n).reshape(n, f_n).astype(np.float32))
+        efs.append(r.uniform(len(s) * f_e).reshape(len(s), f_e).astype(np.float32))
+    y = r.uniform(num_graphs).astype(np.float32) * 0.8 + 0.1
+    return Batch(graphs, np.concatenate(nfs), np.concatenate(efs).reshape(-1, f_e), y,
+                 ["random"] * num_graphs)

@@ -1,0 +1,130 @@
+"""Parameter layout, deterministic initialisation and the weights file.
+
+Layout (SURVEY §8(b) "Weights file"; shapes from P141-P149 read as in
+DESIGN.md R1-R6): for each ANEE layer i = 1..L
+    W_u[d][d_in]  W_e[d][d_e_in]  W_m[d][d]  a_s[d]  a_d[d]
+with d_in = F_n, d_e_in = F_e for i = 1 and d otherwise; then the MLP head
+(P125)  W_1[d_h][d]  b_1[d_h]  w_2[d_h]  b_2[1].
+
+Initialisation: element j of the flat parameter vector (file order) is
+float32((2*u_j - 1) * bound(tensor)), u_j = splitmix64 uniform #j for the
+seed, bound = 1/sqrt(fan_in) (PyTorch-Linear-like).  The C
+library's ``occu_init_weights`` implements the same rule independently.
+
+File: b"OCCUW001", u32[8] = (version=1, L, F_n, F_e, d, d_h, aggr, msg),
+f32 slope, f32 payload (flat, file order), u64 FNV-1a of the payload bytes.
+No method arithmetic lives here.
+"""
+from __future__ import annotations
+
+import math
+import struct
+from dataclasses import dataclass
+
+import numpy as np
+
+from .prng import uniform01
+
+MAGIC = b"OCCUW001"
+VERSION = 1
+AGGR_SUM, AGGR_MEAN = 0, 1
+MSG_CHANNEL_SOFTMAX, MSG_NEIGHBOR_SOFTMAX = 0, 1
+
+
+@dataclass(frozen=True)
+class ModelConfig:
+    L: int = 3
+    F_n: int = 80
+    F_e: int = 4
+    d: int = 128
+    d_h: int = 128
+    aggr: int = AGGR_SUM
+    msg: int = MSG_CHANNEL_SOFTMAX
+    slope: float = 0.01
+
+
+def param_specs(cfg: ModelConfig):
+    """[(name, shape, fan_in)] in file order."""
+    specs = []
+    for i in range(cfg.L):
+        d_in = cfg.F_n if i == 0 else cfg.d
+        de_in = cfg.F_e if i == 0 else cfg.d
+        specs += [
+            (f"W_u{i}", (cfg.d, d_in), d_in),
+            (f"W_e{i}", (cfg.d, de_in), de_in),
+            (f"W_m{i}", (cfg.d, cfg.d), cfg.d),
+            (f"a_s{i}", (cfg.d,), 2 * cfg.d),
+            (f"a_d{i}", (cfg.d,), 2 * cfg.d),
+        ]
+    specs += [
+        ("W_1", (cfg.d_h, cfg.d), cfg.d),
+        ("b_1", (cfg.d_h,), cfg.d),
+        ("w_2", (cfg.d_h,), cfg.d_h),
+        ("b_2", (1,), cfg.d_h),
+    ]
+    return specs
+
+
+def num_params(cfg: ModelConfig) -> int:
+    return sum(int(np.prod(s)) for _, s, _ in param_specs(cfg))
+
+
+def init_flat(cfg: ModelConfig, seed: int) -> np.ndarray:
+    """Flat float32 parameter vector, deterministic in ``seed``."""
+    specs = param_specs(cfg)
+    out = np.empty(num_params(cfg), dtype=np.float32)
+    off = 0
+    for _, shape, fan_in in specs:
+        n = int(np.prod(shape))
+        u = uniform01(seed, n, off)
+        bound = 1.0 / math.sqrt(float(fan_in))
+        out[off:off + n] = ((2.0 * u - 1.0) * bound).astype(np.float32)
+        off += n
+    return out
+
+
+def unflatten(cfg: ModelConfig, flat: np.ndarray) -> dict:
+    out, off = {}, 0
+    for name, shape, _ in param_specs(cfg):
+        n = int(np.prod(shape))
+        out[name] = flat[off:off + n].reshape(shape)
+        off += n
+    assert off == flat.size
+    return out
+
+
+def flatten(cfg: ModelConfig, params: dict) -> np.ndarray:
+    return np.concatenate([np.asarray(params[n], dtype=np.float32).ravel()
+                           for n, _, _ in param_specs(cfg)])
+
+
+def fnv1a64(data: bytes) -> int:
+    h = 0xCBF29CE484222325
+    arr = np.frombuffer(data, dtype=np.uint8)
+    # chunked pure-python loop is slow for 0.5 MB; vectorise per byte sequentially
+    for b in arr.tobytes():
+        h ^= b
+        h = (h * 0x100000001B3) & 0xFFFFFFFFFFFFFFFF
+    return h
+
+
+def write_weights(path: str, cfg: ModelConfig, flat: np.ndarray) -> None:
+    flat = np.ascontiguousarray(flat, dtype="<f4")
+    assert flat.size == num_params(cfg)
+    payload = flat.tobytes()
+    with open(path, "wb") as f:
+        f.write(MAGIC)
+        f.write(struct.pack("<8I", VERSION, cfg.L, cfg.F_n, cfg.F_e, cfg.d, cfg.d_h,
+                            cfg.aggr, cfg.msg))
+        f.write(struct.pack("<f", cfg.slope))
+        f.write(payload)
+        f.write(struct.pack("<Q", fnv1a64(payload)))
+
+
+def unit_scale(cfg: ModelConfig, flat: np.ndarray) -> np.ndarray:
+    """parity weights with W_u multiplied by d so activations keep
+    their scale through the channel softmax (reading A)."""
+    p = unflatten(cfg, flat.copy())
+    for i in range(cfg.L):
+        p[f"W_u{i}"] = (p[f"W_u{i}"].astype(np.float64) * cfg.d).astype(np.float32)
+    return flatten(cfg, p)

@@ -1,0 +1,330 @@
+"""CPU ORACLE for DNN-occu's batched ANEE GNN hot path — TEST INFRASTRUCTURE ONLY.
+
+Only ``tests/``, ``__graft_entry__.smoke()`` and ``bench.py``'s cpu_baseline /
+``--impl reference`` legs may import this module.  The product path (the C-ABI
+library in ``paper_conf_cluster_meiqsgls23_b200/``) never calls it, and this
+module imports nothing from the product package.
+
+Plain NumPy, float64 throughout (the paper fixes no precision).  Every function
+cites the passage it follows; "P<n>" = /root/reference/PAPER.md line n, "R<k>"
+= reading k listed in DESIGN.md §3 (readings of garbled / silent passages).
+
+Computation (per ANEE layer i, P139-P151; R1-R9):
+    h̄   = LeakyReLU(h^{i-1} W_u^T)                                 P141
+    α_l = a_s·h̄_s + a_d·h̄_d   for edge l = (s, d)                  P145, P147 (R1)
+    e^i_l = σ(α_l · (W_e e^{i-1}_l))                                P145 (R2, R3)
+    f(u',l') = Softmax_channels(W_m e^i_l') ⊙ h̄_u'                  P149 (R4, reading A)
+    h^i_u = LeakyReLU(Σ_{l'=(u',u)} f(u',l'))                       P149 (R8, R9)
+then per-graph mean readout (north_star; R11) and the MLP head (P125; R12),
+MSE loss (P209-P213), Adam (P273; R16).
+
+Parity status: every function here is pinned by tests in tests/test_oracle.py
+(hand-derived toy DAGs, closed forms, invariances, finite differences, an
+independent torch-autograd implementation, Adam's first-step closed form).
+"""
+from __future__ import annotations
+
+import struct
+
+import numpy as np
+
+AGGR_SUM, AGGR_MEAN = 0, 1
+MSG_CHANNEL_SOFTMAX, MSG_NEIGHBOR_SOFTMAX = 0, 1
+
+
+# --------------------------------------------------------------------------
+# Step P: packing (P49 "DAG", P139 edge l = (u_s, u_d), P149 Σ over l'=(u',u);
+# tie-break keys are reading R17).  Integer work: must match the library
+# bit for bit.
+# --------------------------------------------------------------------------
+def pack(graphs):
+    """graphs: list of (num_nodes, src[m], dst[m]) with local ids.
+
+    Returns dict of int32 arrays: node_off, edge_off [B+1]; in_ptr [N+1],
+    in_src, in_dst, in_eid [E] (edges sorted by key (dst, src, eid));
+    out_ptr [N+1], out_pos [E] (edges sorted by key (src, dst, eid); out_pos[j]
+    is the in-CSR position of the j-th out-ordered edge); node_graph [N].
+    """
+    B = len(graphs)
+    n_b = np.array([int(g[0]) for g in graphs], dtype=np.int64)
+    m_b = np.array([len(g[1]) for g in graphs], dtype=np.int64)
+    node_off = np.concatenate([[0], np.cumsum(n_b)]).astype(np.int64)
+    edge_off = np.concatenate([[0], np.cumsum(m_b)]).astype(np.int64)
+    N, E = int(node_off[-1]), int(edge_off[-1])
+    src = np.zeros(E, np.int64)
+    dst = np.zeros(E, np.int64)
+    for b, (n, s, t) in enumerate(graphs):
+        src[edge_off[b]:edge_off[b + 1]] = node_off[b] + np.asarray(s, np.int64)
+        dst[edge_off[b]:edge_off[b + 1]] = node_off[b] + np.asarray(t, np.int64)
+    eid = np.arange(E, dtype=np.int64)
+    in_order = np.lexsort((eid, src, dst))        # primary dst, then src, then eid
+    out_order = np.lexsort((eid, dst, src))       # primary src, then dst, then eid
+    in_pos_of_eid = np.empty(E, np.int64)
+    in_pos_of_eid[in_order] = np.arange(E)
+    in_ptr = np.searchsorted(dst[in_order], np.arange(N + 1), side="left")
+    out_ptr = np.searchsorted(src[out_order], np.arange(N + 1), side="left")
+    node_graph = np.repeat(np.arange(B), n_b)
+    i32 = lambda a: np.asarray(a, dtype=np.int32)
+    return {
+        "num_graphs": B, "num_nodes": N, "num_edges": E,
+        "node_off": i32(node_off), "edge_off": i32(edge_off),
+        "in_ptr": i32(in_ptr), "in_src": i32(src[in_order]), "in_dst": i32(dst[in_order]),
+        "in_eid": i32(in_order), "out_ptr": i32(out_ptr),
+        "out_pos": i32(in_pos_of_eid[out_order]), "node_graph": i32(node_graph),
+    }
+
+
+# --------------------------------------------------------------------------
+# Weights file; the oracle reads it with its own reader.
+# --------------------------------------------------------------------------
+def read_weights(path):
+    with open(path, "rb") as f:
+        raw = f.read()
+    if raw[:8] != b"OCCUW001":
+        raise ValueError("bad magic")
+    version, L, F_n, F_e, d, d_h, aggr, msg = struct.unpack_from("<8I", raw, 8)
+    (slope,) = struct.unpack_from("<f", raw, 40)
+    cfg = dict(L=L, F_n=F_n, F_e=F_e, d=d, d_h=d_h, aggr=aggr, msg=msg, slope=float(slope))
+    flat = np.frombuffer(raw, dtype="<f4", offset=44, count=(len(raw) - 52) // 4)
+    return cfg, unflatten(cfg, flat.astype(np.float64))
+
+
+def param_shapes(cfg):
+    """File order; shapes follow P141-P149 (R1, R5) and P125 (R12)."""
+    out = []
+    for i in range(cfg["L"]):
+        d_in = cfg["F_n"] if i == 0 else cfg["d"]
+        de_in = cfg["F_e"] if i == 0 else cfg["d"]
+        out += [(f"W_u{i}", (cfg["d"], d_in)), (f"W_e{i}", (cfg["d"], de_in)),
+                (f"W_m{i}", (cfg["d"], cfg["d"])), (f"a_s{i}", (cfg["d"],)),
+                (f"a_d{i}", (cfg["d"],))]
+    out += [("W_1", (cfg["d_h"], cfg["d"])), ("b_1", (cfg["d_h"],)),
+            ("w_2", (cfg["d_h"],)), ("b_2", (1,))]
+    return out
+
+
+def unflatten(cfg, flat):
+    params, off = {}, 0
+    for name, shape in param_shapes(cfg):
+        n = int(np.prod(shape))
+        params[name] = np.array(flat[off:off + n], dtype=np.float64).reshape(shape)
+        off += n
+    if off != len(flat):
+        raise ValueError("weights payload size mismatch")
+    return params
+
+
+def flatten(cfg, params):
+    return np.concatenate([np.asarray(params[n], np.float64).ravel()
+                           for n, _ in param_shapes(cfg)])
+
+
+# --------------------------------------------------------------------------
+# Elementwise functions (R3 σ = logistic; R7 LeakyReLU slope 0.01).
+# --------------------------------------------------------------------------
+def leaky_relu(x, slope):
+    return np.where(x > 0, x, slope * x)
+
+
+def leaky_relu_grad(x, slope):
+    """PyTorch convention: derivative at 0 is the negative slope (R7)."""
+    return np.where(x > 0, 1.0, slope)
+
+
+def sigmoid(x):
+    return 1.0 / (1.0 + np.exp(-x))
+
+
+def softmax_channels(v):
+    """Softmax over the last axis (channels) of each row: reading A of P149 (R4)."""
+    mx = v.max(axis=-1, keepdims=True)
+    ex = np.exp(v - mx)
+    return ex / ex.sum(axis=-1, keepdims=True)
+
+
+def segment_sum(values, seg_ids, num_segments):
+    """Σ of rows per segment, rows added in ascending row order (np.add.at is
+    sequential and unbuffered).  Empty segments give 0 (R8)."""
+    out = np.zeros((num_segments,) + values.shape[1:], dtype=values.dtype)
+    np.add.at(out, seg_ids, values)
+    return out
+
+
+# --------------------------------------------------------------------------
+# Step F: forward (P141-P151), readout (north_star, R11), head (P125, R12).
+# --------------------------------------------------------------------------
+def anee_layer(params, i, cfg, pk, h_prev, e_prev):
+    """One ANEE round i (0-based) on the packed batch; edges in in-CSR order.
+
+    Returns the layer's intermediates (all float64).
+    """
+    slope = cfg["slope"]
+    s_k, t_k = pk["in_src"].astype(np.int64), pk["in_dst"].astype(np.int64)
+    N = pk["num_nodes"]
+    W_u, W_e, W_m = params[f"W_u{i}"], params[f"W_e{i}"], params[f"W_m{i}"]
+    a_s, a_d = params[f"a_s{i}"], params[f"a_d{i}"]
+    # P141: h̄_u = LeakyReLU(W_u × h_u^{i-1})
+    P = h_prev @ W_u.T
+    hbar = leaky_relu(P, slope)
+    # P145/P147 (R1): a^T (h̄_s || h̄_d) = a_s·h̄_s + a_d·h̄_d, a scalar per edge
+    p = hbar @ a_s
+    q = hbar @ a_d
+    alpha = p[s_k] + q[t_k]
+    # P145 (R2): e_l^i = σ(α_l · (W_e × e_l^{i-1}))
+    z = e_prev @ W_e.T
+    e = sigmoid(alpha[:, None] * z)
+    if cfg.get("msg", MSG_CHANNEL_SOFTMAX) == MSG_CHANNEL_SOFTMAX:
+        # P149 (R4 reading A): f(u',l') = Softmax(W_m × e_l'^i) ⊙ h̄_u'
+        v = e @ W_m.T
+        g = softmax_channels(v)
+        msg = g * hbar[s_k]
+        # P149: h_u^i = LeakyReLU(Σ_{l'=(u',u)} f(u',l'))
+        A = segment_sum(msg, t_k, N)
+    else:
+        # NEXT-1 reading B: per-channel softmax over the in-edges of u
+        v = e @ W_m.T
+        M = np.full((N, v.shape[1]), -np.inf)
+        np.maximum.at(M, t_k, v)
+        ex = np.exp(v - M[t_k])
+        den = segment_sum(ex, t_k, N)
+        g = ex / den[t_k]
+        msg = g * hbar[s_k]
+        A = segment_sum(msg, t_k, N)
+    deg = np.diff(pk["in_ptr"].astype(np.int64))
+    if cfg["aggr"] == AGGR_MEAN:
+        A = A / np.maximum(deg, 1)[:, None]
+    h = leaky_relu(A, slope)
+    return dict(P=P, hbar=hbar, p=p, q=q, alpha=alpha, z=z, e=e, v=v, g=g, A=A, h=h)
+
+
+def forward(params, cfg, pk, node_feat, edge_feat):
+    """Full forward.  node_feat [N,F_n] in graph-concatenated order; edge_feat
+    [E,F_e] in INPUT edge order (permuted to in-CSR order here, step a1)."""
+    h = np.asarray(node_feat, np.float64)
+    e = np.asarray(edge_feat, np.float64)[pk["in_eid"].astype(np.int64)]
+    layers = []
+    for i in range(cfg["L"]):
+        lay = anee_layer(params, i, cfg, pk, h, e)
+        layers.append(lay)
+        h, e = lay["h"], lay["e"]
+    n_b = np.diff(pk["node_off"].astype(np.int64))
+    # north_star: segmented per-graph readout, mean over nodes (R11)
+    r = segment_sum(h, pk["node_graph"].astype(np.int64), pk["num_graphs"]) / n_b[:, None]
+    # P125 MLP head (R12): c = W_1 r + b_1 ; o = LReLU(c) ; ŷ = w_2·o + b_2
+    c = r @ params["W_1"].T + params["b_1"]
+    o = leaky_relu(c, cfg["slope"])
+    yhat = o @ params["w_2"] + params["b_2"][0]
+    return dict(layers=layers, e0=np.asarray(edge_feat, np.float64)[pk["in_eid"].astype(np.int64)],
+                h0=np.asarray(node_feat, np.float64), r=r, c=c, o=o, yhat=yhat)
+
+
+def predict(params, cfg, graphs, node_feat, edge_feat):
+    return forward(params, cfg, pack(graphs), node_feat, edge_feat)["yhat"]
+
+
+# --------------------------------------------------------------------------
+# Step a9: MSE loss (P209-P213), normalised by the GLOBAL batch (R15).
+# --------------------------------------------------------------------------
+def mse_loss(yhat, y, global_batch=None):
+    nb = len(yhat) if global_batch is None else global_batch
+    return float(np.sum((np.asarray(yhat, np.float64) - np.asarray(y, np.float64)) ** 2) / nb)
+
+
+# --------------------------------------------------------------------------
+# Step BW: hand-derived backward of the forward above (reading A), float64.
+# --------------------------------------------------------------------------
+def backward(params, cfg, pk, fwd, y, global_batch=None):
+    slope = cfg["slope"]
+    B = pk["num_graphs"]
+    nb = B if global_batch is None else global_batch
+    s_k, t_k = pk["in_src"].astype(np.int64), pk["in_dst"].astype(np.int64)
+    N = pk["num_nodes"]
+    grads = {}
+    # loss and head
+    dy = 2.0 * (fwd["yhat"] - np.asarray(y, np.float64)) / nb
+    grads["w_2"] = fwd["o"].T @ dy
+    grads["b_2"] = np.array([dy.sum()])
+    dc = (dy[:, None] * params["w_2"][None, :]) * leaky_relu_grad(fwd["c"], slope)
+    grads["W_1"] = dc.T @ fwd["r"]
+    grads["b_1"] = dc.sum(axis=0)
+    dr = dc @ params["W_1"]
+    n_b = np.diff(pk["node_off"].astype(np.int64))
+    gidx = pk["node_graph"].astype(np.int64)
+    dh = dr[gidx] / n_b[gidx][:, None]
+    de_out = None
+    deg = np.diff(pk["in_ptr"].astype(np.int64))
+    for i in range(cfg["L"] - 1, -1, -1):
+        lay = fwd["layers"][i]
+        h_prev = fwd["layers"][i - 1]["h"] if i > 0 else fwd["h0"]
+        e_prev = fwd["layers"][i - 1]["e"] if i > 0 else fwd["e0"]
+        W_u, W_e, W_m = params[f"W_u{i}"], params[f"W_e{i}"], params[f"W_m{i}"]
+        a_s, a_d = params[f"a_s{i}"], params[f"a_d{i}"]
+        hbar, g, e, z, alpha = lay["hbar"], lay["g"], lay["e"], lay["z"], lay["alpha"]
+        dA = dh * leaky_relu_grad(lay["A"], slope)
+        if cfg["aggr"] == AGGR_MEAN:
+            dA = dA / np.maximum(deg, 1)[:, None]
+        dm = dA[t_k]
+        dg = dm * hbar[s_k]
+        dhbar = segment_sum(dm * g, s_k, N)
+        if cfg.get("msg", MSG_CHANNEL_SOFTMAX) == MSG_CHANNEL_SOFTMAX:
+            dv = g * (dg - np.sum(g * dg, axis=1, keepdims=True))
+        else:
+            # segmented (over in-edges of t, per channel) softmax backward
+            dv = g * (dg - segment_sum(g * dg, t_k, N)[t_k])
+        grads[f"W_m{i}"] = dv.T @ e
+        de = dv @ W_m                      # de_k = W_m^T dv_k
+        if de_out is not None:
+            de = de + de_out
+        dyk = de * e * (1.0 - e)
+        dalpha = np.sum(dyk * z, axis=1)
+        dz = alpha[:, None] * dyk
+        grads[f"W_e{i}"] = dz.T @ e_prev
+        de_out = dz @ W_e
+        dp = segment_sum(dalpha, s_k, N)
+        dq = segment_sum(dalpha, t_k, N)
+        grads[f"a_s{i}"] = hbar.T @ dp
+        grads[f"a_d{i}"] = hbar.T @ dq
+        dhbar = dhbar + dp[:, None] * a_s[None, :] + dq[:, None] * a_d[None, :]
+        dP = dhbar * leaky_relu_grad(lay["P"], slope)
+        grads[f"W_u{i}"] = dP.T @ h_prev
+        dh = dP @ W_u
+    loss = mse_loss(fwd["yhat"], y, nb)
+    return loss, grads
+
+
+def loss_and_grads(params, cfg, graphs, node_feat, edge_feat, y, global_batch=None):
+    pk = pack(graphs)
+    fwd = forward(params, cfg, pk, node_feat, edge_feat)
+    return backward(params, cfg, pk, fwd, y, global_batch)
+
+
+# --------------------------------------------------------------------------
+# Step O: Adam (P273 "default hyperparameters", lr = weight decay = 1e-4; R16:
+# PyTorch torch.optim.Adam semantics, L2 weight decay added to the gradient).
+# --------------------------------------------------------------------------
+def adam_step(params, grads, state, lr, wd=1e-4, beta1=0.9, beta2=0.999, eps=1e-8):
+    """Returns (new_params, new_state); state = dict(t, m{name}, v{name})."""
+    t = state.get("t", 0) + 1
+    new_p, m_new, v_new = {}, {}, {}
+    for name, w in params.items():
+        gr = grads[name] + wd * w
+        m = beta1 * state.get("m", {}).get(name, np.zeros_like(w)) + (1 - beta1) * gr
+        v = beta2 * state.get("v", {}).get(name, np.zeros_like(w)) + (1 - beta2) * gr * gr
+        mhat = m / (1 - beta1 ** t)
+        vhat = v / (1 - beta2 ** t)
+        new_p[name] = w - lr * mhat / (np.sqrt(vhat) + eps)
+        m_new[name], v_new[name] = m, v
+    return new_p, {"t": t, "m": m_new, "v": v_new}
+
+
+# --------------------------------------------------------------------------
+# Metrics (P247-P253), used by examples/eval only.
+# --------------------------------------------------------------------------
+def mre(yhat, y):
+    yhat, y = np.asarray(yhat, np.float64), np.asarray(y, np.float64)
+    return float(np.mean(np.abs((yhat - y) / y)))
+
+
+def mse(yhat, y):
+    yhat, y = np.asarray(yhat, np.float64), np.asarray(y, np.float64)
+    return float(np.mean((yhat - y) ** 2))

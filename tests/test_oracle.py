@@ -1,0 +1,406 @@
+"""Pins for the CPU oracle (oracle/occu_oracle.py) — things fixed by the paper's
+equations and by mathematics, not by the oracle itself.
+
+* T1/T2/T3: toy DAGs worked out by hand from P141-P149 (derivations inline,
+  expected decimals also in tests/golden/toy_examples.json).
+* closed forms: a = 0 => e ≡ σ(0) = 1/2; W_m = 0 => g ≡ 1/d; path counts
+  H^i = (A^T)^i X / d^i; d = 1 => ŷ independent of edge data; sources => 0;
+  W_u = 0 => head closed form; reading B on chains => LReLU(h̄_src).
+* invariances: node relabelling, batching, DP sharding of gradients.
+* backward: central finite differences (float64) and an independent torch
+  autograd implementation of the same forward.
+* Adam: first-step closed form and torch.optim.Adam trajectory.
+"""
+import json
+import math
+import os
+
+import numpy as np
+import pytest
+
+import oracle
+from occu_gen import configs, dags, weights
+
+GOLDEN = os.path.join(os.path.dirname(__file__), "golden", "toy_examples.json")
+
+
+def cfg_dict(L=1, F_n=2, F_e=2, d=2, d_h=2, aggr=0, msg=0, slope=0.01):
+    return dict(L=L, F_n=F_n, F_e=F_e, d=d, d_h=d_h, aggr=aggr, msg=msg, slope=slope)
+
+
+def toy_params(cfg, **over):
+    p = {}
+    for name, shape in oracle.param_shapes(cfg):
+        p[name] = np.zeros(shape)
+    p.update(over)
+    return p
+
+
+def sig(x):
+    return 1.0 / (1.0 + math.exp(-x))
+
+
+CHAIN = [(3, np.array([0, 1], np.int32), np.array([1, 2], np.int32))]
+X_T1 = np.array([[1, 2], [3, 4], [5, 6]], np.float64)
+EF_T1 = np.array([[0.1, 0.2], [0.3, 0.4]], np.float64)
+
+
+def t1_params(cfg):
+    return toy_params(cfg, W_u0=np.eye(2), W_e0=np.eye(2), W_m0=np.array([[1., 0.], [0., 0.]]),
+                      W_1=np.eye(2), w_2=np.array([1., 1.]))
+
+
+# ---------------------------------------------------------------- toy DAGs
+def test_T1_chain_alpha_zero():
+    cfg = cfg_dict()
+    f = oracle.forward(t1_params(cfg), cfg, oracle.pack(CHAIN), X_T1, EF_T1)
+    lay = f["layers"][0]
+    # a = 0 -> α = 0 -> e = σ(0) = 1/2 on every channel (P145)
+    assert np.array_equal(lay["e"], np.full((2, 2), 0.5))
+    # W_m e = (1/2, 0) -> channel softmax = (σ(1/2), 1 - σ(1/2))  (P149 reading A)
+    g0 = sig(0.5)
+    assert np.allclose(lay["g"], [[g0, 1 - g0], [g0, 1 - g0]], rtol=0, atol=1e-15)
+    # node 0 has no in-edge -> 0; node1 <- g ⊙ h̄0; node2 <- g ⊙ h̄1 (all positive)
+    h1 = np.array([[0, 0], [g0 * 1, (1 - g0) * 2], [g0 * 3, (1 - g0) * 4]])
+    assert np.allclose(lay["h"], h1, rtol=0, atol=1e-15)
+    r = h1.mean(axis=0)
+    assert np.allclose(f["r"][0], r, atol=1e-15)
+    assert abs(f["yhat"][0] - r.sum()) < 1e-14
+    gold = json.load(open(GOLDEN))["T1"]
+    assert abs(f["yhat"][0] - gold["yhat"]) < 1e-9
+    assert np.allclose(lay["h"], gold["h1"], atol=1e-9)
+
+
+def test_T2_chain_alpha_nonzero():
+    cfg = cfg_dict()
+    p = t1_params(cfg)
+    p.update(a_s0=np.array([1., 0.]), a_d0=np.array([0., 1.]), W_m0=np.eye(2))
+    f = oracle.forward(p, cfg, oracle.pack(CHAIN), X_T1, EF_T1)
+    lay = f["layers"][0]
+    # p = h̄[:,0] = (1,3,5), q = h̄[:,1] = (2,4,6); α(0->1) = 1+4, α(1->2) = 3+6
+    assert np.array_equal(lay["alpha"], [5.0, 9.0])
+    e = np.array([[sig(0.5), sig(1.0)], [sig(2.7), sig(3.6)]])
+    assert np.allclose(lay["e"], e, atol=1e-15)
+    # 2-channel softmax of (x, y) = (σ(x - y), σ(y - x))
+    g = np.array([[sig(e[0, 0] - e[0, 1]), sig(e[0, 1] - e[0, 0])],
+                  [sig(e[1, 0] - e[1, 1]), sig(e[1, 1] - e[1, 0])]])
+    h1 = np.array([[0, 0], [g[0, 0] * 1, g[0, 1] * 2], [g[1, 0] * 3, g[1, 1] * 4]])
+    assert np.allclose(lay["h"], h1, atol=1e-14)
+    gold = json.load(open(GOLDEN))["T2"]
+    assert abs(f["yhat"][0] - gold["yhat"]) < 1e-9
+    assert np.allclose(lay["h"], gold["h1"], atol=1e-9)
+
+
+def test_T3_diamond_path_counts():
+    cfg = cfg_dict(L=2)
+    g = [(4, np.array([0, 0, 1, 2], np.int32), np.array([1, 2, 3, 3], np.int32))]
+    X = np.array([[1, 1], [0, 0], [0, 0], [0, 0]], np.float64)
+    p = toy_params(cfg, W_u0=np.eye(2), W_u1=np.eye(2), W_1=np.eye(2), w_2=np.ones(2))
+    f = oracle.forward(p, cfg, oracle.pack(g), X, np.zeros((4, 2)))
+    assert np.array_equal(f["layers"][0]["h"], [[0, 0], [.5, .5], [.5, .5], [0, 0]])
+    assert np.array_equal(f["layers"][1]["h"], [[0, 0], [0, 0], [0, 0], [.5, .5]])
+
+
+def test_batching_T1_plus_pair():
+    g2 = (2, np.array([0], np.int32), np.array([1], np.int32))
+    pk = oracle.pack(CHAIN + [g2])
+    assert pk["node_off"].tolist() == [0, 3, 5]
+    assert pk["edge_off"].tolist() == [0, 2, 3]
+    cfg = cfg_dict()
+    X = np.vstack([X_T1, [[7, 8], [9, 10]]])
+    EF = np.vstack([EF_T1, [[0.5, 0.6]]])
+    yb = oracle.forward(t1_params(cfg), cfg, pk, X, EF)["yhat"]
+    y1 = oracle.forward(t1_params(cfg), cfg, oracle.pack(CHAIN), X_T1, EF_T1)["yhat"]
+    assert yb[0] == y1[0]
+
+
+# ---------------------------------------------------------------- pack
+def brute_pack_check(graphs, pk):
+    N, E = pk["num_nodes"], pk["num_edges"]
+    src, dst = [], []
+    off = 0
+    for n, s, t in graphs:
+        src += (np.asarray(s) + off).tolist()
+        dst += (np.asarray(t) + off).tolist()
+        off += n
+    trip = sorted(zip(dst, src, range(E)))
+    assert pk["in_dst"].tolist() == [t for t, _, _ in trip]
+    assert pk["in_src"].tolist() == [s for _, s, _ in trip]
+    assert pk["in_eid"].tolist() == [e for _, _, e in trip]
+    for v in range(N + 1):
+        assert pk["in_ptr"][v] == sum(1 for t in dst if t < v)
+        assert pk["out_ptr"][v] == sum(1 for s in src if s < v)
+    otrip = sorted(zip(src, dst, range(E)))
+    for j, (s, t, e) in enumerate(otrip):
+        k = pk["out_pos"][j]
+        assert pk["in_eid"][k] == e and pk["in_src"][k] == s and pk["in_dst"][k] == t
+    assert sorted(pk["out_pos"].tolist()) == list(range(E))
+    ng = []
+    for b, (n, _, _) in enumerate(graphs):
+        ng += [b] * n
+    assert pk["node_graph"].tolist() == ng
+
+
+@pytest.mark.parametrize("seed", range(6))
+def test_pack_brute_force(seed):
+    b = configs.random_dag_batch(7, seed, max_nodes=9, hub=(seed % 2 == 1))
+    # add a multi-edge and an edgeless graph
+    graphs = b.graphs + [(3, np.array([0, 0, 1], np.int32), np.array([2, 2, 2], np.int32)),
+                         (1, np.zeros(0, np.int32), np.zeros(0, np.int32))]
+    pk = oracle.pack(graphs)
+    brute_pack_check(graphs, pk)
+    for k in ("in_ptr", "in_src", "in_eid", "out_ptr", "out_pos", "node_off"):
+        assert pk[k].dtype == np.int32
+
+
+# ---------------------------------------------------------------- closed forms
+def rand_params(cfg, seed, scale=1.0):
+    c = weights.ModelConfig(L=cfg["L"], F_n=cfg["F_n"], F_e=cfg["F_e"], d=cfg["d"],
+                            d_h=cfg["d_h"], aggr=cfg["aggr"], msg=cfg["msg"])
+    flat = weights.init_flat(c, seed).astype(np.float64) * scale
+    return oracle.unflatten(cfg, flat)
+
+
+@pytest.mark.parametrize("seed", range(4))
+def test_path_count_closed_form(seed):
+    """W_u = I (F_n = d), a = 0, W_m = 0, SUM, X >= 0:  H^i = (A^T)^i X / d^i."""
+    d, L = 4, 3
+    cfg = cfg_dict(L=L, F_n=d, F_e=3, d=d, d_h=d)
+    b = configs.random_dag_batch(3, 100 + seed, max_nodes=10, f_n=d, f_e=3, hub=True)
+    X = np.floor(b.node_feat.astype(np.float64) * 8)
+    p = rand_params(cfg, seed)
+    for i in range(L):
+        p[f"W_u{i}"] = np.eye(d)
+        p[f"a_s{i}"] = np.zeros(d)
+        p[f"a_d{i}"] = np.zeros(d)
+        p[f"W_m{i}"] = np.zeros((d, d))
+    pk = oracle.pack(b.graphs)
+    f = oracle.forward(p, cfg, pk, X, b.edge_feat)
+    N = pk["num_nodes"]
+    # brute-force path counts: paths[i][u][v] = # length-i paths u -> v
+    adj = np.zeros((N, N), np.int64)
+    for s, t in zip(pk["in_src"], pk["in_dst"]):
+        adj[s, t] += 1
+    cnt = np.eye(N, dtype=np.int64)
+    for i in range(L):
+        cnt = cnt @ adj
+        expect = cnt.T.astype(np.float64) @ X / d ** (i + 1)
+        assert np.array_equal(f["layers"][i]["h"], expect)
+        assert np.array_equal(f["layers"][i]["e"], np.full((pk["num_edges"], d), 0.5))
+        assert np.array_equal(f["layers"][i]["g"], np.full((pk["num_edges"], d), 1.0 / d))
+
+
+def test_sources_are_zero_and_d1_independent_of_edges():
+    cfg = cfg_dict(L=2, F_n=5, F_e=3, d=1, d_h=3)
+    b = configs.random_dag_batch(5, 9, f_n=5, f_e=3)
+    p = rand_params(cfg, 3, scale=3.0)
+    pk = oracle.pack(b.graphs)
+    f1 = oracle.forward(p, cfg, pk, b.node_feat, b.edge_feat)
+    f2 = oracle.forward(p, cfg, pk, b.node_feat, b.edge_feat * 5.0 + 1.0)
+    assert np.array_equal(f1["yhat"], f2["yhat"])           # softmax of 1 element is 1
+    deg = np.diff(pk["in_ptr"])
+    for lay in f1["layers"]:
+        assert (lay["h"][deg == 0] == 0).all()
+
+
+def test_head_closed_form_when_W_u_zero():
+    cfg = cfg_dict(L=2, F_n=6, F_e=4, d=4, d_h=3)
+    b = configs.random_dag_batch(4, 2, f_n=6, f_e=4)
+    p = rand_params(cfg, 5)
+    p["W_u0"] = np.zeros_like(p["W_u0"])
+    p["W_u1"] = np.zeros_like(p["W_u1"])
+    f = oracle.forward(p, cfg, oracle.pack(b.graphs), b.node_feat, b.edge_feat)
+    b1 = p["b_1"]
+    o = np.where(b1 > 0, b1, 0.01 * b1)
+    assert np.allclose(f["yhat"], o @ p["w_2"] + p["b_2"][0], rtol=0, atol=1e-15)
+
+
+def test_mean_equals_sum_on_chains_and_halves_diamond():
+    cfg_s = cfg_dict(L=2, F_n=3, F_e=2, d=3, d_h=2)
+    cfg_m = dict(cfg_s, aggr=oracle.AGGR_MEAN)
+    chain = [(5, np.arange(4, dtype=np.int32), np.arange(1, 5, dtype=np.int32))]
+    X = np.arange(15, dtype=np.float64).reshape(5, 3) / 7
+    EF = np.arange(8, dtype=np.float64).reshape(4, 2) / 5
+    p = rand_params(cfg_s, 4, 2.0)
+    ys = oracle.forward(p, cfg_s, oracle.pack(chain), X, EF)["yhat"]
+    ym = oracle.forward(p, cfg_m, oracle.pack(chain), X, EF)["yhat"]
+    assert np.array_equal(ys, ym)
+    cfg = cfg_dict(L=2, aggr=oracle.AGGR_MEAN)
+    g = [(4, np.array([0, 0, 1, 2], np.int32), np.array([1, 2, 3, 3], np.int32))]
+    X = np.array([[1, 1], [0, 0], [0, 0], [0, 0]], np.float64)
+    pp = toy_params(cfg, W_u0=np.eye(2), W_u1=np.eye(2))
+    f = oracle.forward(pp, cfg, oracle.pack(g), X, np.zeros((4, 2)))
+    assert np.array_equal(f["layers"][1]["h"][3], [.25, .25])   # mean of two (.25,.25)
+
+
+def test_reading_B_chain_closed_form():
+    """NEXT-1 reading B: a single in-edge has weight 1 => h_t = LReLU(h̄_src)."""
+    cfg = cfg_dict(L=1, F_n=3, F_e=2, d=4, d_h=2, msg=oracle.MSG_NEIGHBOR_SOFTMAX)
+    chain = [(4, np.arange(3, dtype=np.int32), np.arange(1, 4, dtype=np.int32))]
+    X = np.arange(12, dtype=np.float64).reshape(4, 3) / 5 - 1
+    p = rand_params(cfg, 8, 3.0)
+    lay = oracle.forward(p, cfg, oracle.pack(chain), X, np.ones((3, 2)))["layers"][0]
+    hb = lay["hbar"]
+    expect = np.vstack([np.zeros(4), np.where(hb[:3] > 0, hb[:3], 0.01 * hb[:3])])
+    assert np.allclose(lay["h"], expect, rtol=0, atol=1e-15)
+
+
+# ---------------------------------------------------------------- invariances
+@pytest.mark.parametrize("msg", [0, 1])
+def test_node_permutation_invariance(msg):
+    cfg = cfg_dict(L=3, F_n=80, F_e=4, d=16, d_h=16, msg=msg)
+    b = configs.random_dag_batch(4, 21, max_nodes=15, hub=True)
+    p = rand_params(cfg, 11)
+    for i in range(3):
+        p[f"W_u{i}"] *= 16
+    y0 = oracle.predict(p, cfg, b.graphs, b.node_feat, b.edge_feat)
+    from occu_gen.prng import Rng
+    r = Rng(77)
+    graphs, feats = [], []
+    off = 0
+    for (n, s, t) in b.graphs:
+        perm = r.permutation(n)
+        inv = np.argsort(perm)
+        graphs.append((n, perm[s].astype(np.int32), perm[t].astype(np.int32)))
+        feats.append(b.node_feat[off:off + n][inv])
+        off += n
+    y1 = oracle.predict(p, cfg, graphs, np.vstack(feats), b.edge_feat)
+    assert np.allclose(y0, y1, rtol=1e-12, atol=0)
+
+
+def test_batching_invariance_bitwise():
+    cfg = cfg_dict(L=3, F_n=80, F_e=4, d=8, d_h=8)
+    b = configs.random_dag_batch(6, 31, max_nodes=12, hub=True)
+    p = rand_params(cfg, 2)
+    yb = oracle.predict(p, cfg, b.graphs, b.node_feat, b.edge_feat)
+    for i in range(b.num_graphs):
+        s = b.subset([i])
+        yi = oracle.predict(p, cfg, s.graphs, s.node_feat, s.edge_feat)
+        assert np.allclose(yi[0], yb[i], rtol=1e-13, atol=1e-15)
+
+
+# ---------------------------------------------------------------- backward
+def fd_check(cfg, b, p, names=None, eps_rel=1e-5, tol=2e-6, gb=None):
+    """Central differences.  Bound: truncation O(h^2) (relative tol) plus the
+    round-off of differencing two float64 losses, ~eps_mach*|loss|/h per entry."""
+    pk = oracle.pack(b.graphs)
+    loss, grads = oracle.backward(p, cfg, pk, oracle.forward(p, cfg, pk, b.node_feat, b.edge_feat),
+                                  b.targets, gb)
+    names = names or list(p)
+    for name in names:
+        w = p[name]
+        flat = w.ravel()
+        num = np.zeros_like(flat)
+        hmin = np.inf
+        for j in range(flat.size):
+            h = eps_rel * max(1.0, abs(flat[j]))
+            hmin = min(hmin, h)
+            old = flat[j]
+            flat[j] = old + h
+            lp = oracle.mse_loss(oracle.forward(p, cfg, pk, b.node_feat, b.edge_feat)["yhat"], b.targets, gb)
+            flat[j] = old - h
+            lm = oracle.mse_loss(oracle.forward(p, cfg, pk, b.node_feat, b.edge_feat)["yhat"], b.targets, gb)
+            flat[j] = old
+            num[j] = (lp - lm) / (2 * h)
+        an = grads[name].ravel()
+        roundoff = 50 * np.finfo(np.float64).eps * abs(loss) / hmin * np.sqrt(flat.size)
+        err = np.linalg.norm(an - num)
+        assert err <= tol * np.linalg.norm(num) + roundoff, (name, err, np.linalg.norm(num), roundoff)
+        # the gradient must not be vacuous for the weights that matter
+    assert any(np.linalg.norm(grads[n]) > 1e-3 for n in names)
+
+
+@pytest.mark.parametrize("d,L,aggr,msg", [(2, 1, 0, 0), (4, 2, 0, 0), (4, 2, 1, 0), (3, 2, 0, 1)])
+def test_backward_finite_differences(d, L, aggr, msg):
+    cfg = cfg_dict(L=L, F_n=5, F_e=3, d=d, d_h=3, aggr=aggr, msg=msg)
+    b = configs.random_dag_batch(3, 40 + d, max_nodes=7, f_n=5, f_e=3, hub=True)
+    p = rand_params(cfg, 6, scale=2.0)
+    for i in range(L):
+        p[f"W_u{i}"] *= d
+    fd_check(cfg, b, p, tol=2e-6)
+
+
+def torch_forward_loss(p, cfg, pk, X, EF, y):
+    torch = pytest.importorskip("torch")
+    T = {k: torch.tensor(v, dtype=torch.float64, requires_grad=True) for k, v in p.items()}
+    s = torch.tensor(pk["in_src"].astype(np.int64))
+    t = torch.tensor(pk["in_dst"].astype(np.int64))
+    h = torch.tensor(X, dtype=torch.float64)
+    e = torch.tensor(EF, dtype=torch.float64)[torch.tensor(pk["in_eid"].astype(np.int64))]
+    lrelu = lambda x: torch.nn.functional.leaky_relu(x, cfg["slope"])
+    N = pk["num_nodes"]
+    for i in range(cfg["L"]):
+        hb = lrelu(h @ T[f"W_u{i}"].T)
+        al = hb[s] @ T[f"a_s{i}"] + hb[t] @ T[f"a_d{i}"]
+        e = torch.sigmoid(al[:, None] * (e @ T[f"W_e{i}"].T))
+        g = torch.softmax(e @ T[f"W_m{i}"].T, dim=1)
+        A = torch.zeros(N, hb.shape[1], dtype=torch.float64).index_add(0, t, g * hb[s])
+        if cfg["aggr"] == 1:
+            A = A / torch.tensor(np.maximum(np.diff(pk["in_ptr"]), 1), dtype=torch.float64)[:, None]
+        h = lrelu(A)
+        ng = torch.tensor(pk["node_graph"].astype(np.int64))
+    nb = torch.tensor(np.diff(pk["node_off"]).astype(np.float64))
+    r = torch.zeros(pk["num_graphs"], h.shape[1], dtype=torch.float64).index_add(0, ng, h) / nb[:, None]
+    yh = lrelu(r @ T["W_1"].T + T["b_1"]) @ T["w_2"] + T["b_2"][0]
+    loss = ((yh - torch.tensor(y, dtype=torch.float64)) ** 2).sum() / len(y)
+    loss.backward()
+    return float(loss), {k: v.grad.numpy() for k, v in T.items()}
+
+
+@pytest.mark.parametrize("aggr", [0, 1])
+def test_backward_matches_torch_autograd(aggr):
+    cfg = cfg_dict(L=3, F_n=80, F_e=4, d=16, d_h=8, aggr=aggr)
+    b = configs.random_dag_batch(5, 50, max_nodes=14, hub=True)
+    p = rand_params(cfg, 13)
+    for i in range(3):
+        p[f"W_u{i}"] *= 16
+    pk = oracle.pack(b.graphs)
+    loss, grads = oracle.backward(p, cfg, pk, oracle.forward(p, cfg, pk, b.node_feat, b.edge_feat),
+                                  b.targets)
+    tl, tg = torch_forward_loss(p, cfg, pk, b.node_feat, b.edge_feat, b.targets)
+    assert abs(loss - tl) <= 1e-12 * abs(tl)
+    for k in p:
+        assert np.allclose(grads[k], tg[k], rtol=1e-9, atol=1e-14 * max(1, np.abs(tg[k]).max())), k
+
+
+def test_dp_shard_gradients_sum_to_full_batch():
+    cfg = cfg_dict(L=2, F_n=80, F_e=4, d=8, d_h=8)
+    b = configs.random_dag_batch(8, 60, max_nodes=10)
+    p = rand_params(cfg, 17)
+    B = b.num_graphs
+    _, g_full = oracle.loss_and_grads(p, cfg, b.graphs, b.node_feat, b.edge_feat, b.targets)
+    acc = {k: np.zeros_like(v) for k, v in p.items()}
+    for shard in ([0, 3, 5], [1, 2], [4, 6, 7]):
+        s = b.subset(shard)
+        _, gs = oracle.loss_and_grads(p, cfg, s.graphs, s.node_feat, s.edge_feat, s.targets, B)
+        for k in acc:
+            acc[k] += gs[k]
+    for k in p:
+        assert np.allclose(acc[k], g_full[k], rtol=1e-12, atol=1e-16), k
+
+
+# ---------------------------------------------------------------- Adam
+def test_adam_first_step_closed_form():
+    rng = np.random.default_rng(0)
+    p = {"w": rng.normal(size=20)}
+    g = {"w": rng.normal(size=20) * 1e-3}
+    lr, wd, eps = 1e-4, 1e-4, 1e-8
+    newp, st = oracle.adam_step(p, g, {}, lr, wd)
+    gh = g["w"] + wd * p["w"]
+    assert np.allclose(newp["w"], p["w"] - lr * gh / (np.abs(gh) + eps), rtol=0, atol=1e-15)
+    assert st["t"] == 1
+
+
+def test_adam_matches_torch_optim():
+    torch = pytest.importorskip("torch")
+    rng = np.random.default_rng(1)
+    w0 = rng.normal(size=(5, 3))
+    grads = [rng.normal(size=(5, 3)) for _ in range(6)]
+    tw = torch.tensor(w0, dtype=torch.float64, requires_grad=True)
+    opt = torch.optim.Adam([tw], lr=1e-3, weight_decay=1e-4)
+    p, st = {"w": w0.copy()}, {}
+    for g in grads:
+        tw.grad = torch.tensor(g, dtype=torch.float64)
+        opt.step()
+        p, st = oracle.adam_step(p, {"w": g}, st, 1e-3, 1e-4)
+    assert np.allclose(p["w"], tw.detach().numpy(), rtol=1e-12, atol=1e-15)
