@@ -1,0 +1,400 @@
+#!/usr/bin/env python
+"""Benchmark of the DNN-occu GNN hot path (BASELINE.json metric: GNN graphs/sec,
+infer & train; aggregation HBM GB/s vs peak).
+
+Workload (N=1 headline): BASELINE.json configs[1] = CFG2, 256 ResNet-50 training
+graphs (hyperparameter variants), 3-layer ANEE GNN, hidden 128, inference, FP32.
+A step = one occu_predict over the 256-graph batch (rows a1-a8 of SURVEY §8(a)).
+Weak scaling: each rank processes its own 256-graph shard, no collective
+(north_star: "Inference batches shard by graph with no collective").  The train
+object times occu_train_step on the same batch (forward, loss, backward, NCCL
+gradient allreduce when N > 1, Adam).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+L2_BYTES = 126 * 1024 * 1024
+
+
+def load_peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            p = json.load(f)
+        return p, "measured"
+    except Exception:
+        return {"hbm_gbs": 6650.0, "bf16_tflops": 1590.0, "sm_max_mhz": 1965.0}, "fallback"
+
+
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons sampled during the timed region."""
+
+    Q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index):
+        self.index = index
+        self.proc = None
+        self.lines = []
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.Q}",
+                 "--format=csv,noheader,nounits", "-lms", "100"],
+                stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for ln in self.proc.stdout:
+            self.lines.append(ln.strip())
+
+    def __exit__(self, *a):
+        if self.proc:
+            time.sleep(0.15)
+            self.proc.terminate()
+            try:
+                self.proc.wait(2)
+            except Exception:
+                self.proc.kill()
+
+    def summary(self):
+        sm, mx, reasons = [], 0.0, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            f = [x.strip() for x in ln.split(",")]
+            if len(f) < 7:
+                continue
+            try:
+                sm.append(float(f[0]))
+                mx = max(mx, float(f[1]))
+            except ValueError:
+                continue
+            for n, v in zip(names, f[3:7]):
+                if v.lower().startswith("active"):
+                    reasons.add(n)
+        if not sm:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unsampled"], "samples": 0}
+        return {"sm_mhz": float(np.median(sm)), "sm_max_mhz": mx, "reasons": sorted(reasons),
+                "samples": len(sm)}
+
+
+def dist_env():
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return rank, world, local
+
+
+# ---------------------------------------------------------------- algorithmic bytes
+def aggregation_bytes(N, E, d, s=4):
+    """a5 + a6 (gather_segsum): read g [E,d], gather h̄[src] once per node (perfect
+    L2 reuse), write h [N,d], read in_src/in_ptr."""
+    return s * (E * d + N * d + N * d) + 4 * (E + N + 1)
+
+
+def edge_fwd_flops(E, d, de_in):
+    """a3 + a4: two GEMMs per edge (W_e: 2·de_in·d, W_m: 2·d·d)."""
+    return 2.0 * E * d * (de_in + d)
+
+
+def node_gemm_flops(N, d, d_in):
+    return 2.0 * N * d * d_in
+
+
+def cpu_cores_used():
+    try:
+        from threadpoolctl import threadpool_info
+        n = max([i.get("num_threads", 1) for i in threadpool_info()] or [1])
+        return int(n)
+    except Exception:
+        return len(os.sched_getaffinity(0))
+
+
+def run_reference(args):
+    """--impl reference: the CPU oracle (float64 NumPy) as it stands, on the box's
+    host cores, each step a bounded sample (args.ref_graphs graphs) of CFG2."""
+    rank, world, local = dist_env()
+    if rank != 0:
+        return 0
+    import oracle
+    from occu_gen import configs, weights
+    wc = weights.ModelConfig(L=3, F_n=80, F_e=4, d=128, d_h=128)
+    ocf = dict(L=3, F_n=80, F_e=4, d=128, d_h=128, aggr=0, msg=0, slope=float(np.float32(0.01)))
+    params = oracle.unflatten(ocf, weights.init_flat(wc, 42).astype(np.float64))
+    full = configs.cfg2(256)
+    G = args.ref_graphs
+    times = []
+    for it in range(args.warmup + args.steps):
+        idx = [(it * G + j) % 256 for j in range(G)]
+        s = full.subset(idx)
+        t0 = time.perf_counter()
+        oracle.predict(params, ocf, s.graphs, s.node_feat, s.edge_feat)
+        dt = time.perf_counter() - t0
+        if it >= args.warmup:
+            times.append(dt)
+    tot = sum(times)
+    value = G * len(times) / tot
+    cores = cpu_cores_used()
+    line = {
+        "metric": "GNN graphs/sec (inference, CFG2: ResNet-50 training graphs x256, L=3, d=128)",
+        "value": value, "unit": "graphs/s", "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": 1e3 * tot / len(times), "higher_is_better": True,
+        "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+        "impl": "reference",
+        "config": {"workload": "CFG2 sample", "graphs_per_step": G, "L": 3, "d": 128},
+        "cpu_baseline": {"value": value, "unit": "graphs/s", "cores": cores, "kind": "oracle",
+                         "sample": f"{G} CFG2 graphs per step, float64 NumPy oracle forward"},
+        "e2e": {"value": value, "unit": "graphs/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+def cpu_baseline_sample(seconds=12.0):
+    """The oracle as it stands on a bounded CFG2 sample, graphs/s."""
+    import oracle
+    from occu_gen import configs, weights
+    wc = weights.ModelConfig(L=3, F_n=80, F_e=4, d=128, d_h=128)
+    ocf = dict(L=3, F_n=80, F_e=4, d=128, d_h=128, aggr=0, msg=0, slope=float(np.float32(0.01)))
+    params = oracle.unflatten(ocf, weights.init_flat(wc, 42).astype(np.float64))
+    full = configs.cfg2(256)
+    done, t0 = 0, time.perf_counter()
+    while time.perf_counter() - t0 < seconds and done < 256:
+        s = full.subset([done, done + 1])
+        oracle.predict(params, ocf, s.graphs, s.node_feat, s.edge_feat)
+        done += 2
+    dt = time.perf_counter() - t0
+    return {"value": done / dt, "unit": "graphs/s", "cores": cpu_cores_used(), "kind": "oracle",
+            "sample": f"{done} CFG2 ResNet-50 graphs (L=3, d=128), float64 NumPy oracle forward, "
+                      f"{dt:.1f} s"}
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--graphs", type=int, default=256, help="graphs per rank per step (CFG2: 256)")
+    ap.add_argument("--ref-graphs", type=int, default=32)
+    ap.add_argument("--no-train", action="store_true")
+    ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--no-flush", action="store_true")
+    args = ap.parse_args()
+    if args.warmup < 3:
+        args.warmup = 3
+    if args.impl == "reference":
+        return run_reference(args)
+
+    import torch
+    rank, world, local = dist_env()
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    pg = None
+    if world > 1:
+        import torch.distributed as dist
+        dist.init_process_group("nccl", device_id=dev)
+        pg = dist
+    from occu_gen import configs, weights
+    from paper_conf_cluster_meiqsgls23_b200 import build as pkg_build
+    from paper_conf_cluster_meiqsgls23_b200 import occu
+
+    if rank == 0:
+        pkg_build.build()
+    if pg:
+        pg.barrier()
+    peaks, peak_src = load_peaks()
+    c = occu.config(L=3, F_n=80, F_e=4, d=128)
+    stream = torch.cuda.current_stream(dev)
+    model = occu.Model(c, device=local, stream=stream.cuda_stream)
+    model.init_weights(42)
+    batch = configs.cfg2(args.graphs)              # every rank: its own CFG2 shard (weak)
+    B, N, E = batch.num_graphs, batch.num_nodes, batch.num_edges
+    host_csr = occu.pack(batch.graphs)
+    csr = model.to_device(host_csr)
+    nf = torch.from_numpy(batch.node_feat).to(dev)
+    ef = torch.from_numpy(batch.edge_feat).to(dev)
+    yt = torch.from_numpy(batch.targets).to(dev)
+    out = torch.empty(B, dtype=torch.float32, device=dev)
+    flush = torch.empty(2 * L2_BYTES // 4, dtype=torch.float32, device=dev)
+
+    def timed(fn, steps, profile=False):
+        """Per-step CUDA events on the launch stream; L2 flushed between steps."""
+        ms = []
+        launches = 0
+        if profile:
+            model.profile_reset()
+            model.set_profiling(True)
+        for _ in range(steps):
+            if not args.no_flush:
+                flush.fill_(1.0)
+            a = torch.cuda.Event(enable_timing=True)
+            b = torch.cuda.Event(enable_timing=True)
+            a.record(stream)
+            fn()
+            b.record(stream)
+            launches += model.last_launch_count()
+            ms.append((a, b))
+        torch.cuda.synchronize()
+        if profile:
+            model.set_profiling(False)
+        return [x.elapsed_time(y) for x, y in ms], launches
+
+    def bar():
+        if pg:
+            pg.barrier()
+        torch.cuda.synchronize()
+
+    def max_over_ranks(v):
+        if not pg:
+            return v
+        t = torch.tensor([v], dtype=torch.float64, device=dev)
+        pg.all_reduce(t, op=pg.ReduceOp.MAX)
+        return float(t.item())
+
+    infer = lambda: model.predict(csr, nf, ef, out)
+    # ---- inference (headline)
+    timed(infer, args.warmup)
+    bar()
+    with ClockSampler(local) as clk:
+        times, launches = timed(infer, args.steps, profile=True)
+    bar()
+    prof = model.profile()
+    ms_step = max_over_ranks(float(np.sum(times)) / args.steps)
+    value = B * world / (ms_step * 1e-3)
+
+    # roofline: per-kernel device time inside the timed region (CUDA events)
+    d = 128
+    tot_kernel = sum(v[0] for v in prof.values())
+    shares = {k: v[0] / max(tot_kernel, 1e-9) for k, v in prof.items()}
+    dom = max(prof, key=lambda k: prof[k][0])
+
+    def kernel_avg_ms(name):
+        t, n = prof.get(name, (0.0, 0))
+        return t / max(n, 1)
+
+    agg_bytes_per_launch = aggregation_bytes(N, E, d)
+    agg_ms = kernel_avg_ms("gather_segsum")
+    agg = {"kernel": "gather_segsum", "bound": "hbm",
+           "achieved": agg_bytes_per_launch / (agg_ms * 1e-3) / 1e9 if agg_ms else None,
+           "peak": peaks["hbm_gbs"], "unit": "GB/s",
+           "algorithmic_bytes_per_launch": agg_bytes_per_launch, "avg_ms": agg_ms}
+    agg["frac"] = agg["achieved"] / agg["peak"] if agg["achieved"] else None
+    agg["frac_of_8TBps"] = agg["achieved"] / 8000.0 if agg["achieved"] else None
+    # FP32 SIMT GEMM kernels are FP32-ALU bound: peak = 148 SMs x 128 FMA/clk x 2 x max clock
+    alu_peak_tflops = 148 * 128 * 2 * peaks.get("sm_max_mhz", 1965.0) * 1e6 / 1e12
+    if dom == "edge_fwd":
+        # per launch: layer 1 (de_in = 4) and layers 2-3 (de_in = d): average over the 3 launches
+        fl = (edge_fwd_flops(E, d, 4) + 2 * edge_fwd_flops(E, d, d)) / 3
+        roof = {"kernel": dom, "bound": "alu", "achieved": fl / (kernel_avg_ms(dom) * 1e-3) / 1e12,
+                "peak": alu_peak_tflops, "unit": "TFLOP/s", "traffic": None,
+                "peak_source": "DESIGN.md §6: 148 SM x 128 FP32 lanes x 2 x 1965 MHz"}
+    elif dom == "node_gemm":
+        fl = (node_gemm_flops(N, d, 80) + 2 * node_gemm_flops(N, d, d)) / 3
+        roof = {"kernel": dom, "bound": "alu", "achieved": fl / (kernel_avg_ms(dom) * 1e-3) / 1e12,
+                "peak": alu_peak_tflops, "unit": "TFLOP/s", "traffic": None,
+                "peak_source": "DESIGN.md §6: 148 SM x 128 FP32 lanes x 2 x 1965 MHz"}
+    else:
+        roof = {"kernel": "gather_segsum", "bound": "hbm", "achieved": agg["achieved"],
+                "peak": peaks["hbm_gbs"], "unit": "GB/s", "traffic": None}
+    roof["frac"] = roof["achieved"] / roof["peak"] if roof["achieved"] else None
+    roof["peak_kind"] = peak_src
+    roof["share_of_step"] = shares.get(roof["kernel"])
+
+    # ---- e2e through the public API with host buffers (pinned), pack included
+    pin_nf = torch.from_numpy(batch.node_feat).pin_memory()
+    pin_ef = torch.from_numpy(batch.edge_feat).pin_memory()
+    pin_out = torch.empty(B, dtype=torch.float32).pin_memory()
+    graphs = batch.graphs
+
+    def e2e_step():
+        hc = occu.pack(graphs)
+        model.predict(hc, pin_nf, pin_ef, pin_out)
+        return hc
+
+    for _ in range(args.warmup):
+        e2e_step()
+    bar()
+    t0 = time.perf_counter()
+    for _ in range(args.steps):
+        e2e_step()
+    torch.cuda.synchronize()
+    e2e_ms = max_over_ranks((time.perf_counter() - t0) * 1e3 / args.steps)
+    csr_bytes = 4 * (2 * (B + 1) + 2 * (N + 1) + 4 * E + N)
+    e2e = {"value": B * world / (e2e_ms * 1e-3), "unit": "graphs/s", "ms_per_step": e2e_ms,
+           "h2d_bytes_per_step": int(batch.node_feat.nbytes + batch.edge_feat.nbytes + csr_bytes),
+           "d2h_bytes_per_step": int(B * 4),
+           "includes": "occu_pack (host C++) + occu_predict with pinned host buffers (H2D, kernels, D2H)"}
+
+    # ---- training step (DP over graphs, NCCL allreduce inside the library when N > 1)
+    train = None
+    if not args.no_train:
+        if pg and world > 1:
+            uid = [occu.Model.nccl_unique_id() if rank == 0 else None]
+            pg.broadcast_object_list(uid, src=0)
+            model.dist_init(rank, world, uid[0])
+        gB = B * world
+        step = lambda: model.train_step(csr, nf, ef, yt, 1e-4, global_num_graphs=gB, want_loss=False)
+        timed(step, args.warmup)
+        bar()
+        ttimes, tl = timed(step, args.steps)
+        bar()
+        tms = max_over_ranks(float(np.sum(ttimes)) / args.steps)
+        loss = model.train_step(csr, nf, ef, yt, 1e-4, global_num_graphs=gB)
+        train = {"value": gB / (tms * 1e-3), "unit": "graphs/s", "ms_per_step": tms,
+                 "global_batch": gB, "gpu_launches": tl, "loss_after": loss,
+                 "includes": "forward with saves, MSE, backward, "
+                             + ("NCCL allreduce, " if world > 1 else "") + "Adam"}
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu:
+        cpu = cpu_baseline_sample()
+
+    if rank == 0:
+        line = {
+            "metric": "GNN graphs/sec (inference, CFG2: ResNet-50 training graphs x256, L=3, d=128)",
+            "value": value, "unit": "graphs/s", "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+            "config": {"workload": "CFG2 (BASELINE.json configs[1])", "graphs_per_rank": B,
+                       "nodes_per_rank": N, "edges_per_rank": E, "L": 3, "d": 128, "F_n": 80,
+                       "F_e": 4, "precision": "fp32 (SIMT)",
+                       "l2": "flushed between timed steps (256 MiB write)" if not args.no_flush else "not flushed",
+                       "parallelism": f"graph-sharded x{world}, no collective"},
+            "gpu_launches": launches,
+            "clocks": clk.summary(),
+            "roofline": roof,
+            "aggregation": agg,
+            "kernel_ms_per_step": {k: v[0] / args.steps for k, v in prof.items()},
+            "e2e": e2e,
+            "train": train,
+            "cpu_baseline": cpu,
+        }
+        print(json.dumps(line), flush=True)
+    if pg:
+        pg.barrier()
+        pg.destroy_process_group()
+    return 0
+
+
+if __name__ == "__main__":
+    sys.exit(main())

@@ -1,0 +1,195 @@
+/*
+ * occu.h — C ABI of the B200-native DNN-occu GNN hot path.
+ *
+ * The method (Mei et al., "GPU Occupancy Prediction of Deep Learning Models
+ * Using Graph Neural Network"; PAPER.md = /root/reference/PAPER.md, "P<n>" =
+ * its line n) maps a DL model's computation DAG (P49, P139) with Table I
+ * node/edge features (P97-P133) to one GPU-occupancy scalar (P81, P85-P91):
+ * ANEE message-passing rounds (P139-P151), a per-graph readout and an MLP head
+ * (P125), trained with MSE (P209-P213) and Adam (P273).  Readings of garbled or
+ * silent passages are DESIGN.md §3 R1-R22.
+ *
+ * Conventions (all entry points)
+ *  - Every call returns an occu_status; no C++ exception crosses the ABI.  On a
+ *    non-OK status nothing is written to caller outputs and occu_last_error()
+ *    returns a message for that ctx (or the thread's last ctx-less error).
+ *  - Ownership: the caller owns every input array and output buffer; the
+ *    library borrows them for the duration of the call only.  The library owns
+ *    weights, Adam state, workspace and the NCCL communicator (freed by
+ *    occu_destroy).  occu_csr_batch objects are owned by the library and freed
+ *    with occu_batch_free.
+ *  - Memory space: feature/target/output pointers may be host or device
+ *    (detected with cudaPointerGetAttributes); node_feat, edge_feat and out_occ
+ *    of one call must be in the same space.  Host pointers => the call is
+ *    synchronous.  Device pointers => the call is stream-ordered on the ctx
+ *    stream and returns before completion.
+ *  - Layout: row-major, little-endian float32, 16-byte aligned rows are NOT
+ *    required (F_n = 80, F_e = 4 give 320 B / 16 B rows anyway).
+ *  - Determinism: same inputs + same world size + same precision => bitwise
+ *    identical outputs (no atomics on any reduction; fixed reduction orders).
+ *  - Thread safety: one ctx per host thread.
+ */
+#ifndef OCCU_H_
+#define OCCU_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define OCCU_ABI_VERSION 1
+
+typedef struct occu_ctx occu_ctx;
+
+typedef enum {
+  OCCU_OK = 0,
+  OCCU_EINVAL = 1,    /* bad argument: sizes, ids out of range, self-loop, config mismatch */
+  OCCU_ENOMEM = 2,    /* host or device allocation failed */
+  OCCU_ECUDA = 3,     /* CUDA runtime error (message in occu_last_error) */
+  OCCU_EFORMAT = 4,   /* weights/state file malformed or checksum mismatch */
+  OCCU_ENOTREADY = 5, /* weights not initialised / nothing computed yet */
+  OCCU_ENCCL = 6      /* NCCL error */
+} occu_status;
+
+typedef enum { OCCU_AGGR_SUM = 0, OCCU_AGGR_MEAN = 1 } occu_aggr;            /* P149 Σ; MEAN option */
+typedef enum { OCCU_MSG_CHANNEL_SOFTMAX = 0, OCCU_MSG_NEIGHBOR_SOFTMAX = 1 } occu_msg; /* R4 */
+typedef enum { OCCU_FP32 = 0, OCCU_BF16 = 1 } occu_precision;
+
+/* Model configuration.  L ANEE rounds of width d; raw feature widths F_n
+ * (node, Table I) and F_e (edge); head hidden width d_h; LeakyReLU slope
+ * (R7, 0.01).  d must be a multiple of 32 and <= 256 (kernel tiling);
+ * F_n, F_e multiples of 4.  msg = OCCU_MSG_NEIGHBOR_SOFTMAX is reserved
+ * (NEXT-1) and rejected with OCCU_EINVAL by this build. */
+typedef struct {
+  int32_t L, F_n, F_e, d, d_h;
+  int32_t aggr;      /* occu_aggr */
+  int32_t msg;       /* occu_msg */
+  int32_t prec;      /* occu_precision */
+  float slope;
+} occu_config;
+
+/* One caller-owned input graph (host memory), local node ids. */
+typedef struct {
+  int32_t num_nodes;          /* >= 1 */
+  int32_t num_edges;          /* >= 0 */
+  const int32_t *src, *dst;   /* [num_edges], ids in [0, num_nodes), src != dst */
+} occu_graph_view;
+
+/* Packed batch.  Graphs concatenated in caller order; global
+ * id = node_off[b] + local id; global input edge id = edge_off[b] + j.
+ *   in-CSR : edges sorted by key (dst, src, eid); in_ptr[v] = #{edges with dst < v}
+ *   out-CSR: edges sorted by key (src, dst, eid); out_pos[j] = in-CSR position
+ *            of the j-th out-ordered edge; out_ptr[v] = #{edges with src < v}
+ * All int32.  on_device = 0: host arrays (occu_pack); 1: device arrays
+ * (occu_batch_to_device).  Library-owned; free with occu_batch_free. */
+typedef struct {
+  int32_t num_graphs, num_nodes, num_edges;
+  int32_t *node_off, *edge_off;           /* [B+1] */
+  int32_t *in_ptr;                        /* [N+1] */
+  int32_t *in_src, *in_dst, *in_eid;      /* [E]   */
+  int32_t *out_ptr;                       /* [N+1] */
+  int32_t *out_pos;                       /* [E]   */
+  int32_t *node_graph;                    /* [N]   */
+  int32_t on_device;
+  void *priv;                             /* library-private (device schedule) */
+} occu_csr_batch;
+
+/* Training batch: packed CSR + features (same conventions as occu_predict);
+ * global_num_graphs = B summed over all DP ranks (loss scale 1/B_glob, R15). */
+typedef struct {
+  const occu_csr_batch *csr;
+  const float *node_feat;     /* [N][F_n] graph-concatenated order */
+  const float *edge_feat;     /* [E][F_e] graph-concatenated INPUT edge order */
+  int32_t global_num_graphs;
+} occu_batch;
+
+/* ---- lifecycle ------------------------------------------------------------ */
+/* Create a context on CUDA device `cuda_device`, launching on `cuda_stream`
+ * (a cudaStream_t; NULL = the legacy default stream).  Validates cfg. */
+occu_status occu_create(occu_ctx **out, const occu_config *cfg, int cuda_device, void *cuda_stream);
+occu_status occu_destroy(occu_ctx *ctx);
+/* Rebind the launch stream (e.g. torch's current stream). */
+occu_status occu_set_stream(occu_ctx *ctx, void *cuda_stream);
+size_t occu_num_params(const occu_config *cfg);
+
+/* ---- weights (SURVEY §8(b) file format "OCCUW001") ------------------------ */
+/* Deterministic init: element j of the flat parameter vector (file order) =
+ * float((2u_j - 1) / sqrt(fan_in)), u_j = splitmix64 uniform #j for seed (R21). */
+occu_status occu_init_weights(occu_ctx *ctx, uint64_t seed);
+occu_status occu_load_weights(occu_ctx *ctx, const char *path);    /* EFORMAT on mismatch */
+occu_status occu_save_weights(const occu_ctx *ctx, const char *path);
+/* Flat float32 parameter vector in file order, host memory, n = occu_num_params. */
+occu_status occu_set_params(occu_ctx *ctx, const float *host_flat, size_t n);
+occu_status occu_get_params(const occu_ctx *ctx, float *host_flat, size_t n);
+
+/* ---- packing (host, C++; a0) ---------------------------------------------- */
+/* EINVAL: num_graphs < 1, num_nodes < 1, id out of range, self-loop,
+ * N or E >= 2^31.  Acyclicity is not checked (the math is a fixed number of
+ * rounds).  Threaded over graphs; output is bit-identical to oracle.pack. */
+occu_status occu_pack(const occu_graph_view *graphs, int32_t num_graphs, occu_csr_batch **out);
+/* Device copy (+ kernel schedule) of a host batch, on the ctx stream. */
+occu_status occu_batch_to_device(occu_ctx *ctx, const occu_csr_batch *host, occu_csr_batch **dev_out);
+void occu_batch_free(occu_csr_batch *b);
+
+/* ---- forward (P139-P151, P125) -------------------------------------------- */
+/* out_occ[B] <- ŷ for each graph.  csr_batch host or device. */
+occu_status occu_predict(occu_ctx *ctx, const occu_csr_batch *csr_batch,
+                         const float *node_feat, const float *edge_feat, float *out_occ);
+
+/* ---- training (P209-P213, P273) ------------------------------------------- */
+/* Forward with saved activations, MSE loss scaled by 1/global_num_graphs,
+ * backward, NCCL allreduce of the flat gradient (if occu_dist_init was
+ * called), Adam(lr, wd = 1e-4, β = (0.9, 0.999), ε = 1e-8).  targets[B] in
+ * the features' memory space; out_loss (nullable, host) = global mean loss. */
+occu_status occu_train_step(occu_ctx *ctx, const occu_batch *batch, const float *targets,
+                            float lr, float *out_loss);
+/* Forward + backward only (no allreduce, no Adam): grads left in the ctx. */
+occu_status occu_compute_grads(occu_ctx *ctx, const occu_batch *batch, const float *targets,
+                               float *out_loss);
+occu_status occu_get_grads(const occu_ctx *ctx, float *host_flat, size_t n);
+occu_status occu_set_weight_decay(occu_ctx *ctx, float wd);
+
+/* ---- data parallel (north_star: NCCL gradient allreduce over NVLink) ------ */
+occu_status occu_nccl_unique_id(void *out_128_bytes);
+occu_status occu_dist_init(occu_ctx *ctx, int rank, int world, const void *nccl_unique_id);
+
+/* ---- optimizer state (Adam m, v, t) --------------------------------------- */
+occu_status occu_save_state(const occu_ctx *ctx, const char *path);
+occu_status occu_load_state(occu_ctx *ctx, const char *path);
+
+/* ---- introspection for parity tests --------------------------------------- */
+typedef enum {
+  OCCU_T_HBAR = 0,   /* [N][d]  layer l */
+  OCCU_T_P = 1,      /* [N]     layer l */
+  OCCU_T_Q = 2,      /* [N]     layer l */
+  OCCU_T_E = 3,      /* [E][d]  layer l, in-CSR edge order */
+  OCCU_T_H = 4,      /* [N][d]  layer l */
+  OCCU_T_R = 5,      /* [B][d]  readout */
+  OCCU_T_YHAT = 6    /* [B] */
+} occu_tensor;
+/* Keep every intermediate of the next forward (costs memory/bandwidth). */
+occu_status occu_set_keep_intermediates(occu_ctx *ctx, int keep);
+/* Copy an intermediate of the last forward into host memory (float32; BF16
+ * precision stores are widened).  bytes must equal the tensor size. */
+occu_status occu_get_tensor(occu_ctx *ctx, int32_t which, int32_t layer, void *host_dst, size_t bytes);
+/* Number of kernel launches issued by the last predict/train call. */
+int64_t occu_last_launch_count(const occu_ctx *ctx);
+
+/* ---- per-kernel timing (CUDA events recorded on the ctx stream) ---------- */
+/* enable != 0: every kernel launch is bracketed by a pair of cudaEvents on the
+ * launch stream; occu_profile_query(idx) returns the idx-th kernel name, the
+ * summed device time (ms) and the launch count since the last reset
+ * (synchronises the stream).  EINVAL when idx is out of range. */
+occu_status occu_set_profiling(occu_ctx *ctx, int enable);
+occu_status occu_profile_reset(occu_ctx *ctx);
+occu_status occu_profile_query(occu_ctx *ctx, int32_t idx, const char **name, double *total_ms,
+                               int64_t *launches);
+
+const char *occu_last_error(const occu_ctx *ctx);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* OCCU_H_ */

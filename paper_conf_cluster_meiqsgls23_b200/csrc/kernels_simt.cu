@@ -1,0 +1,982 @@
+// FP32 CUDA-core (SIMT) kernels for the ANEE hot path on sm_100a.
+//
+// Forward, per layer (DESIGN.md §1 rows a2-a6; P141-P151 with readings R1-R9):
+//   node_gemm   : h̄ = LReLU(h W_uᵀ), p = h̄·a_s, q = h̄·a_d                    (a2)
+//   edge_fwd    : z = W_e e ; e' = σ((p[s]+q[t]) z) ; g = softmax_c(W_m e')   (a3, a4)
+//   gather_segsum: h[t] = LReLU(Σ_{k∈seg(t)} g_k ⊙ h̄[s_k])  (warp per node)   (a5, a6)
+// then readout_head (a7, a8).  Backward (a9, a10) and Adam (a12) follow the
+// hand derivation in SURVEY §8(c) "Step BW"; every reduction has a fixed order
+// (no atomics), so results are bitwise reproducible.
+//
+// Tiling: 64-row tiles, 256 threads as 16 (tx) x 16 (ty); thread owns rows
+// ty*4..ty*4+3 and columns {tx*4+j, 64+tx*4+j}.  The whole weight matrix sits
+// in shared memory (d <= 128), persistent CTAs loop over tiles.
+#include <cuda_runtime.h>
+#include <math.h>
+#include <stdint.h>
+
+#include <algorithm>
+
+#include "occu_internal.h"
+
+namespace occu {
+namespace {
+
+constexpr int BM = 64;
+constexpr int NT = 256;
+
+__device__ __forceinline__ float lrelu(float x, float s) { return x > 0.f ? x : s * x; }
+__device__ __forceinline__ float lrelu_grad_from_out(float y, float s) { return y > 0.f ? 1.f : s; }
+__device__ __forceinline__ float sigmoidf_(float x) { return 1.f / (1.f + expf(-x)); }
+
+__device__ __forceinline__ float hsum16(float v) {   // sum over the 16 lanes sharing ty
+  v += __shfl_xor_sync(0xffffffffu, v, 1);
+  v += __shfl_xor_sync(0xffffffffu, v, 2);
+  v += __shfl_xor_sync(0xffffffffu, v, 4);
+  v += __shfl_xor_sync(0xffffffffu, v, 8);
+  return v;
+}
+__device__ __forceinline__ float hmax16(float v) {
+  v = fmaxf(v, __shfl_xor_sync(0xffffffffu, v, 1));
+  v = fmaxf(v, __shfl_xor_sync(0xffffffffu, v, 2));
+  v = fmaxf(v, __shfl_xor_sync(0xffffffffu, v, 4));
+  v = fmaxf(v, __shfl_xor_sync(0xffffffffu, v, 8));
+  return v;
+}
+
+// Column owned by (tx, j): D=128 -> tx*4+j (j<4) and 64+tx*4+(j-4); D=64 -> tx*4+j.
+template <int D> __device__ __forceinline__ int colof(int tx, int j) {
+  return (j < 4) ? tx * 4 + j : 64 + tx * 4 + (j - 4);
+}
+template <int D> struct Tn { static constexpr int v = D / 16; };
+
+// Load W into smem as Ws[k][n] (row length D).  TRANS: W is [D][K] and
+// Ws[k][n] = W[n][k] (for y = x Wᵀ); otherwise W is [K][D] and Ws = W.
+template <int D, bool TRANS>
+__device__ void load_weights(float *Ws, const float *__restrict__ W, int K) {
+  if (TRANS) {
+    for (int idx = threadIdx.x; idx < K * D; idx += NT) {
+      const int n = idx / K, k = idx % K;        // coalesced read of W[n][k]
+      Ws[k * D + n] = W[idx];
+    }
+  } else {
+    for (int idx = threadIdx.x; idx < K * D; idx += NT) Ws[idx] = W[idx];
+  }
+}
+
+// Load `rows` x K (row-major, K % 4 == 0) rows starting at row0 into As with
+// row stride S = K + 4; rows beyond `nrows` are zero.
+__device__ void load_rows(float *As, const float *__restrict__ A, long row0, int nrows, int K) {
+  const int S = K + 4, kq = K / 4;
+  for (int idx = threadIdx.x; idx < BM * kq; idx += NT) {
+    const int r = idx / kq, c = (idx % kq) * 4;
+    float4 v = make_float4(0.f, 0.f, 0.f, 0.f);
+    if (r < nrows) v = __ldg(reinterpret_cast<const float4 *>(A + (row0 + r) * K + c));
+    *reinterpret_cast<float4 *>(As + r * S + c) = v;
+  }
+}
+
+// acc[i][j] += Σ_k As[row_i][k] * Ws[k][col_j], rows ty*4+i, K % 4 == 0.
+template <int D>
+__device__ __forceinline__ void gemm_tile(const float *As, int K, const float *Ws,
+                                          float (&acc)[4][Tn<D>::v], int tx, int ty) {
+  constexpr int TN = Tn<D>::v;
+  const int S = K + 4;
+  for (int k = 0; k < K; k += 4) {
+    float4 a[4];
+#pragma unroll
+    for (int i = 0; i < 4; ++i) a[i] = *reinterpret_cast<const float4 *>(As + (ty * 4 + i) * S + k);
+#pragma unroll
+    for (int kk = 0; kk < 4; ++kk) {
+      float b[TN];
+      const float *w = Ws + (k + kk) * D;
+      const float4 b0 = *reinterpret_cast<const float4 *>(w + tx * 4);
+      b[0] = b0.x; b[1] = b0.y; b[2] = b0.z; b[3] = b0.w;
+      if (TN == 8) {
+        const float4 b1 = *reinterpret_cast<const float4 *>(w + 64 + tx * 4);
+        b[4 % TN] = b1.x; b[5 % TN] = b1.y; b[6 % TN] = b1.z; b[7 % TN] = b1.w;
+      }
+#pragma unroll
+      for (int i = 0; i < 4; ++i) {
+        const float av = kk == 0 ? a[i].x : kk == 1 ? a[i].y : kk == 2 ? a[i].z : a[i].w;
+#pragma unroll
+        for (int j = 0; j < TN; ++j) acc[i][j] = fmaf(av, b[j], acc[i][j]);
+      }
+    }
+  }
+}
+
+template <int D> __device__ __forceinline__ void zero_acc(float (&acc)[4][Tn<D>::v]) {
+#pragma unroll
+  for (int i = 0; i < 4; ++i)
+#pragma unroll
+    for (int j = 0; j < Tn<D>::v; ++j) acc[i][j] = 0.f;
+}
+
+// Store a row-slice of 4-column groups (float4) for row r of a [*, D] matrix.
+template <int D>
+__device__ __forceinline__ void store_row(float *dst, const float (&v)[Tn<D>::v], int tx) {
+  *reinterpret_cast<float4 *>(dst + tx * 4) = make_float4(v[0], v[1], v[2], v[3]);
+  if (Tn<D>::v == 8)
+    *reinterpret_cast<float4 *>(dst + 64 + tx * 4) =
+        make_float4(v[4 % Tn<D>::v], v[5 % Tn<D>::v], v[6 % Tn<D>::v], v[7 % Tn<D>::v]);
+}
+template <int D>
+__device__ __forceinline__ void load_row(const float *src, float (&v)[Tn<D>::v], int tx) {
+  const float4 a = __ldg(reinterpret_cast<const float4 *>(src + tx * 4));
+  v[0] = a.x; v[1] = a.y; v[2] = a.z; v[3] = a.w;
+  if (Tn<D>::v == 8) {
+    const float4 b = __ldg(reinterpret_cast<const float4 *>(src + 64 + tx * 4));
+    v[4 % Tn<D>::v] = b.x; v[5 % Tn<D>::v] = b.y; v[6 % Tn<D>::v] = b.z; v[7 % Tn<D>::v] = b.w;
+  }
+}
+
+// ---------------------------------------------------------------------------
+// a2: node transform.  MODE 0: h̄ = LReLU(A Wᵀ), p, q (forward).
+//                      MODE 1: C = A W (plain GEMM, backward dh_prev = dP W_u).
+// ---------------------------------------------------------------------------
+template <int D, int MODE>
+__global__ void __launch_bounds__(NT) node_gemm_kernel(const float *__restrict__ A, int K,
+                                                       const float *__restrict__ W,
+                                                       const float *__restrict__ a_s,
+                                                       const float *__restrict__ a_d, int N,
+                                                       float slope, float *__restrict__ out,
+                                                       float *__restrict__ p,
+                                                       float *__restrict__ q) {
+  extern __shared__ __align__(16) float smem[];
+  float *Ws = smem;                 // [K][D]
+  float *As = Ws + K * D;           // [BM][K+4]
+  constexpr int TN = Tn<D>::v;
+  const int tx = threadIdx.x % 16, ty = threadIdx.x / 16;
+  load_weights<D, MODE == 0>(Ws, W, K);
+  float as_[TN], ad_[TN];
+  if (MODE == 0) {
+#pragma unroll
+    for (int j = 0; j < TN; ++j) {
+      as_[j] = a_s[colof<D>(tx, j)];
+      ad_[j] = a_d[colof<D>(tx, j)];
+    }
+  }
+  const int tiles = (N + BM - 1) / BM;
+  for (int tile = blockIdx.x; tile < tiles; tile += gridDim.x) {
+    const long r0 = long(tile) * BM;
+    const int nrows = min(BM, int(N - r0));
+    __syncthreads();
+    load_rows(As, A, r0, nrows, K);
+    __syncthreads();
+    float acc[4][TN];
+    zero_acc<D>(acc);
+    gemm_tile<D>(As, K, Ws, acc, tx, ty);
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+      const int r = ty * 4 + i;
+      float v[TN];
+      float pp = 0.f, qq = 0.f;
+#pragma unroll
+      for (int j = 0; j < TN; ++j) {
+        v[j] = MODE == 0 ? lrelu(acc[i][j], slope) : acc[i][j];
+        if (MODE == 0) {
+          pp = fmaf(v[j], as_[j], pp);
+          qq = fmaf(v[j], ad_[j], qq);
+        }
+      }
+      if (MODE == 0) {
+        pp = hsum16(pp);
+        qq = hsum16(qq);
+      }
+      if (r < nrows) {
+        store_row<D>(out + (r0 + r) * D, v, tx);
+        if (MODE == 0 && tx == 0) {
+          p[r0 + r] = pp;
+          q[r0 + r] = qq;
+        }
+      }
+    }
+  }
+}
+
+// ---------------------------------------------------------------------------
+// a3 + a4: edge transform and channel softmax gate, edges in in-CSR order.
+// ---------------------------------------------------------------------------
+template <int D>
+__global__ void __launch_bounds__(NT) edge_fwd_kernel(
+    const float *__restrict__ e_in, int Ke, const float *__restrict__ W_e,
+    const float *__restrict__ W_m, const float *__restrict__ p, const float *__restrict__ q,
+    const int32_t *__restrict__ in_src, const int32_t *__restrict__ in_dst, int E,
+    float *__restrict__ e_out, float *__restrict__ g_out) {
+  extern __shared__ __align__(16) float smem[];
+  float *Wes = smem;                // [Ke][D]  (W_eᵀ)
+  float *Wms = Wes + Ke * D;        // [D][D]   (W_mᵀ)
+  float *As = Wms + D * D;          // [BM][Ke+4]
+  float *Es = As + BM * (Ke + 4);   // [BM][D+4]
+  float *alpha = Es + BM * (D + 4); // [BM]
+  constexpr int TN = Tn<D>::v;
+  const int tx = threadIdx.x % 16, ty = threadIdx.x / 16;
+  load_weights<D, true>(Wes, W_e, Ke);
+  load_weights<D, true>(Wms, W_m, D);
+  const int tiles = (E + BM - 1) / BM;
+  for (int tile = blockIdx.x; tile < tiles; tile += gridDim.x) {
+    const long k0 = long(tile) * BM;
+    const int nrows = min(BM, int(E - k0));
+    __syncthreads();
+    load_rows(As, e_in, k0, nrows, Ke);
+    if (threadIdx.x < BM) {
+      const int r = threadIdx.x;
+      alpha[r] = r < nrows ? p[in_src[k0 + r]] + q[in_dst[k0 + r]] : 0.f;   // R1
+    }
+    __syncthreads();
+    float acc[4][TN];
+    zero_acc<D>(acc);
+    gemm_tile<D>(As, Ke, Wes, acc, tx, ty);                                  // z = W_e e
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+      const int r = ty * 4 + i;
+      const float al = alpha[r];
+      float v[TN];
+#pragma unroll
+      for (int j = 0; j < TN; ++j) v[j] = sigmoidf_(al * acc[i][j]);          // e' (R2, R3)
+      store_row<D>(Es + r * (D + 4), v, tx);
+      if (e_out && r < nrows) store_row<D>(e_out + (k0 + r) * D, v, tx);
+    }
+    __syncthreads();
+    zero_acc<D>(acc);
+    gemm_tile<D>(Es, D, Wms, acc, tx, ty);                                   // v = W_m e'
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+      const int r = ty * 4 + i;
+      float mx = -INFINITY;
+#pragma unroll
+      for (int j = 0; j < TN; ++j) mx = fmaxf(mx, acc[i][j]);
+      mx = hmax16(mx);
+      float v[TN], s = 0.f;
+#pragma unroll
+      for (int j = 0; j < TN; ++j) {
+        v[j] = expf(acc[i][j] - mx);
+        s += v[j];
+      }
+      s = hsum16(s);
+#pragma unroll
+      for (int j = 0; j < TN; ++j) v[j] = v[j] / s;                           // g (R4 reading A)
+      if (r < nrows) store_row<D>(g_out + (k0 + r) * D, v, tx);
+    }
+  }
+}
+
+// ---------------------------------------------------------------------------
+// a5 + a6: gather + deterministic segmented sum, warp per destination node.
+// Lane l owns channels [l*V, l*V+V), V = D/32; edges summed in ascending k.
+// ---------------------------------------------------------------------------
+template <int D>
+__global__ void __launch_bounds__(NT) gather_segsum_kernel(
+    const float *__restrict__ g, const float *__restrict__ hbar,
+    const int32_t *__restrict__ in_ptr, const int32_t *__restrict__ in_src, int N, int mean,
+    float slope, float *__restrict__ h_out) {
+  constexpr int V = D / 32;
+  const int lane = threadIdx.x & 31;
+  const int warps = (gridDim.x * NT) / 32;
+  for (int t = (blockIdx.x * NT + threadIdx.x) / 32; t < N; t += warps) {
+    const int beg = in_ptr[t], end = in_ptr[t + 1];
+    float acc[V];
+#pragma unroll
+    for (int c = 0; c < V; ++c) acc[c] = 0.f;
+    for (int base = beg; base < end; base += 32) {
+      const int cnt = min(32, end - base);
+      const int s_l = lane < cnt ? in_src[base + lane] : 0;
+      for (int j = 0; j < cnt; ++j) {
+        const int s = __shfl_sync(0xffffffffu, s_l, j);
+        const float *gr = g + long(base + j) * D + lane * V;
+        const float *hr = hbar + long(s) * D + lane * V;
+        if (V == 4) {
+          const float4 a = __ldg(reinterpret_cast<const float4 *>(gr));
+          const float4 b = __ldg(reinterpret_cast<const float4 *>(hr));
+          acc[0] = fmaf(a.x, b.x, acc[0]);
+          acc[1 % V] = fmaf(a.y, b.y, acc[1 % V]);
+          acc[2 % V] = fmaf(a.z, b.z, acc[2 % V]);
+          acc[3 % V] = fmaf(a.w, b.w, acc[3 % V]);
+        } else {
+#pragma unroll
+          for (int c = 0; c < V; ++c) acc[c] = fmaf(__ldg(gr + c), __ldg(hr + c), acc[c]);
+        }
+      }
+    }
+    const int deg = end - beg;
+#pragma unroll
+    for (int c = 0; c < V; ++c) {
+      float a = acc[c];
+      if (mean) a = a / float(deg > 0 ? deg : 1);
+      h_out[long(t) * D + lane * V + c] = lrelu(a, slope);
+    }
+  }
+}
+
+// e0[k] = edge_feat[in_eid[k]]  (a1)
+__global__ void permute_rows_kernel(const float *__restrict__ src, const int32_t *__restrict__ idx,
+                                    int rows, int width, float *__restrict__ dst) {
+  const long total = long(rows) * width;
+  for (long i = blockIdx.x * long(blockDim.x) + threadIdx.x; i < total;
+       i += long(gridDim.x) * blockDim.x) {
+    const long r = i / width, c = i % width;
+    dst[i] = src[long(idx[r]) * width + c];
+  }
+}
+
+// ---------------------------------------------------------------------------
+// a7 + a8: readout (mean over the graph's nodes, ascending node id per
+// 4-way interleaved partial, partials combined in fixed order) and head.
+// ---------------------------------------------------------------------------
+__global__ void readout_head_kernel(const float *__restrict__ h, const int32_t *__restrict__ node_off,
+                                    int D, int d_h, const float *__restrict__ W_1,
+                                    const float *__restrict__ b_1, const float *__restrict__ w_2,
+                                    const float *__restrict__ b_2, float slope,
+                                    float *__restrict__ r_out, float *__restrict__ c_out,
+                                    float *__restrict__ yhat) {
+  extern __shared__ float sm[];
+  float *part = sm;              // [4][D]
+  float *rs = part + 4 * D;      // [D]
+  float *os = rs + D;            // [d_h]
+  const int b = blockIdx.x;
+  const int u0 = node_off[b], u1 = node_off[b + 1];
+  const int c = threadIdx.x % D, grp = threadIdx.x / D;   // blockDim = 4*D
+  float acc = 0.f;
+  for (int u = u0 + grp; u < u1; u += 4) acc += h[long(u) * D + c];
+  part[grp * D + c] = acc;
+  __syncthreads();
+  if (threadIdx.x < D) {
+    const float s = ((part[c] + part[D + c]) + part[2 * D + c]) + part[3 * D + c];
+    const float rv = s / float(u1 - u0);
+    rs[c] = rv;
+    r_out[long(b) * D + c] = rv;
+  }
+  __syncthreads();
+  for (int j = threadIdx.x; j < d_h; j += blockDim.x) {
+    float cv = 0.f;
+    for (int k = 0; k < D; ++k) cv = fmaf(W_1[long(j) * D + k], rs[k], cv);
+    cv += b_1[j];
+    c_out[long(b) * d_h + j] = cv;
+    os[j] = lrelu(cv, slope);
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    float y = 0.f;
+    for (int j = 0; j < d_h; ++j) y = fmaf(w_2[j], os[j], y);
+    yhat[b] = y + b_2[0];
+  }
+}
+
+// ---------------------------------------------------------------------------
+// Backward.
+// ---------------------------------------------------------------------------
+// Per graph: dŷ_b = 2(ŷ_b - y_b)/B_glob ; dc = dŷ w_2 ⊙ LReLU'(c) ; dr = W_1ᵀ dc
+__global__ void head_bwd_graph_kernel(const float *__restrict__ yhat, const float *__restrict__ y,
+                                      const float *__restrict__ c, const float *__restrict__ W_1,
+                                      const float *__restrict__ w_2, int D, int d_h, float inv_gb,
+                                      float slope, float *__restrict__ dy, float *__restrict__ dc,
+                                      float *__restrict__ dr) {
+  extern __shared__ float sm[];
+  const int b = blockIdx.x;
+  const float d = 2.f * (yhat[b] - y[b]) * inv_gb;
+  for (int j = threadIdx.x; j < d_h; j += blockDim.x) {
+    const float cv = c[long(b) * d_h + j];
+    const float v = d * w_2[j] * (cv > 0.f ? 1.f : slope);
+    sm[j] = v;
+    dc[long(b) * d_h + j] = v;
+  }
+  if (threadIdx.x == 0) dy[b] = d;
+  __syncthreads();
+  for (int k = threadIdx.x; k < D; k += blockDim.x) {
+    float s = 0.f;
+    for (int j = 0; j < d_h; ++j) s = fmaf(W_1[long(j) * D + k], sm[j], s);
+    dr[long(b) * D + k] = s;
+  }
+}
+
+// Head parameter gradients and the loss, each a fixed-order sum over graphs.
+__global__ void head_bwd_reduce_kernel(const float *__restrict__ dy, const float *__restrict__ dc,
+                                       const float *__restrict__ r, const float *__restrict__ c,
+                                       const float *__restrict__ yhat, const float *__restrict__ y,
+                                       int B, int D, int d_h, float inv_gb, float slope,
+                                       float *__restrict__ gW_1, float *__restrict__ gb_1,
+                                       float *__restrict__ gw_2, float *__restrict__ gb_2,
+                                       float *__restrict__ loss) {
+  const int jobs = d_h * D + 2 * d_h + 2;
+  for (int t = blockIdx.x * blockDim.x + threadIdx.x; t < jobs; t += gridDim.x * blockDim.x) {
+    float s = 0.f;
+    if (t < d_h * D) {
+      const int j = t / D, k = t % D;
+      for (int b = 0; b < B; ++b) s = fmaf(dc[long(b) * d_h + j], r[long(b) * D + k], s);
+      gW_1[t] = s;
+    } else if (t < d_h * D + d_h) {
+      const int j = t - d_h * D;
+      for (int b = 0; b < B; ++b) s += dc[long(b) * d_h + j];
+      gb_1[j] = s;
+    } else if (t < d_h * D + 2 * d_h) {
+      const int j = t - d_h * D - d_h;
+      for (int b = 0; b < B; ++b) s = fmaf(dy[b], lrelu(c[long(b) * d_h + j], slope), s);
+      gw_2[j] = s;
+    } else if (t == d_h * D + 2 * d_h) {
+      for (int b = 0; b < B; ++b) s += dy[b];
+      gb_2[0] = s;
+    } else {
+      for (int b = 0; b < B; ++b) {
+        const float e = yhat[b] - y[b];
+        s = fmaf(e, e, s);
+      }
+      loss[0] = s * inv_gb;
+    }
+  }
+}
+
+// dh^L_u = dr_{graph(u)} / n_{graph(u)}
+__global__ void broadcast_dh_kernel(const float *__restrict__ dr, const int32_t *__restrict__ node_graph,
+                                    const int32_t *__restrict__ node_off, int N, int D,
+                                    float *__restrict__ dh) {
+  const long total = long(N) * D;
+  for (long i = blockIdx.x * long(blockDim.x) + threadIdx.x; i < total;
+       i += long(gridDim.x) * blockDim.x) {
+    const int u = int(i / D), k = int(i % D);
+    const int b = node_graph[u];
+    dh[i] = dr[long(b) * D + k] / float(node_off[b + 1] - node_off[b]);
+  }
+}
+
+// Edge backward, phase A (W_m): recompute g = softmax(W_m e'), then
+//   dm = dA[t] ; dg = dm ⊙ h̄[s] ; MG = dm ⊙ g ; dv = g ⊙ (dg - <g,dg>) ;
+//   de = W_mᵀ dv + de_out.
+// dA[t] = dh[t] ⊙ LReLU'(A_t) (÷ deg for MEAN); sign(A) = sign(h).
+template <int D>
+__global__ void __launch_bounds__(NT) edge_bwd_m_kernel(
+    const float *__restrict__ e, const float *__restrict__ W_m, const float *__restrict__ hbar,
+    const float *__restrict__ h, const float *__restrict__ dh, const float *__restrict__ de_out,
+    const int32_t *__restrict__ in_src, const int32_t *__restrict__ in_dst,
+    const int32_t *__restrict__ in_ptr, int E, int mean, float slope,
+    float *__restrict__ MG, float *__restrict__ DV, float *__restrict__ de) {
+  extern __shared__ __align__(16) float smem[];
+  float *WmT = smem;               // [D][D] W_mᵀ
+  float *Wm = WmT + D * D;         // [D][D] W_m
+  float *As = Wm + D * D;          // [BM][D+4]
+  int *sidx = reinterpret_cast<int *>(As + BM * (D + 4));   // [BM] src
+  int *tidx = sidx + BM;                                      // [BM] dst
+  constexpr int TN = Tn<D>::v;
+  const int tx = threadIdx.x % 16, ty = threadIdx.x / 16;
+  load_weights<D, true>(WmT, W_m, D);
+  load_weights<D, false>(Wm, W_m, D);
+  const int tiles = (E + BM - 1) / BM;
+  for (int tile = blockIdx.x; tile < tiles; tile += gridDim.x) {
+    const long k0 = long(tile) * BM;
+    const int nrows = min(BM, int(E - k0));
+    __syncthreads();
+    load_rows(As, e, k0, nrows, D);
+    if (threadIdx.x < BM) {
+      const int r = threadIdx.x;
+      sidx[r] = r < nrows ? in_src[k0 + r] : 0;
+      tidx[r] = r < nrows ? in_dst[k0 + r] : 0;
+    }
+    __syncthreads();
+    float acc[4][TN];
+    zero_acc<D>(acc);
+    gemm_tile<D>(As, D, WmT, acc, tx, ty);
+    float dv[4][TN];
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+      const int r = ty * 4 + i;
+      float mx = -INFINITY;
+#pragma unroll
+      for (int j = 0; j < TN; ++j) mx = fmaxf(mx, acc[i][j]);
+      mx = hmax16(mx);
+      float gg[TN], s = 0.f;
+#pragma unroll
+      for (int j = 0; j < TN; ++j) {
+        gg[j] = expf(acc[i][j] - mx);
+        s += gg[j];
+      }
+      s = hsum16(s);
+#pragma unroll
+      for (int j = 0; j < TN; ++j) gg[j] = gg[j] / s;
+      const int t = tidx[r], sr = sidx[r];
+      float dhv[TN], hv[TN], hb[TN];
+      load_row<D>(dh + long(t) * D, dhv, tx);
+      load_row<D>(h + long(t) * D, hv, tx);
+      load_row<D>(hbar + long(sr) * D, hb, tx);
+      float inv = 1.f;
+      if (mean) {
+        const int deg = in_ptr[t + 1] - in_ptr[t];
+        inv = float(deg > 0 ? deg : 1);
+      }
+      float mg[TN], dg[TN], dot = 0.f;
+#pragma unroll
+      for (int j = 0; j < TN; ++j) {
+        float dm = dhv[j] * lrelu_grad_from_out(hv[j], slope);
+        if (mean) dm = dm / inv;
+        dg[j] = dm * hb[j];
+        mg[j] = dm * gg[j];
+        dot = fmaf(gg[j], dg[j], dot);
+      }
+      dot = hsum16(dot);
+#pragma unroll
+      for (int j = 0; j < TN; ++j) dv[i][j] = gg[j] * (dg[j] - dot);
+      if (r < nrows) {
+        store_row<D>(MG + (k0 + r) * D, mg, tx);
+        store_row<D>(DV + (k0 + r) * D, dv[i], tx);
+      }
+    }
+    __syncthreads();   // everyone done reading As (e') -> reuse for dv
+#pragma unroll
+    for (int i = 0; i < 4; ++i) store_row<D>(As + (ty * 4 + i) * (D + 4), dv[i], tx);
+    __syncthreads();
+    zero_acc<D>(acc);
+    gemm_tile<D>(As, D, Wm, acc, tx, ty);                    // W_mᵀ dv (row form dv W_m)
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+      const int r = ty * 4 + i;
+      if (r >= nrows) continue;
+      float v[TN];
+      if (de_out) {
+        float o[TN];
+        load_row<D>(de_out + (k0 + r) * D, o, tx);
+#pragma unroll
+        for (int j = 0; j < TN; ++j) v[j] = acc[i][j] + o[j];
+      } else {
+#pragma unroll
+        for (int j = 0; j < TN; ++j) v[j] = acc[i][j];
+      }
+      store_row<D>(de + (k0 + r) * D, v, tx);
+    }
+  }
+}
+
+// Edge backward, phase B (W_e): dy = de ⊙ e'(1-e') ; z = W_e e_in (recompute) ;
+// dα = <dy, z> ; dz = α dy ; de_prev = W_eᵀ dz (layer > 0).
+template <int D>
+__global__ void __launch_bounds__(NT) edge_bwd_e_kernel(
+    const float *__restrict__ e_in, int Ke, const float *__restrict__ e, const float *__restrict__ de,
+    const float *__restrict__ W_e, const float *__restrict__ p, const float *__restrict__ q,
+    const int32_t *__restrict__ in_src, const int32_t *__restrict__ in_dst, int E,
+    float *__restrict__ DZ, float *__restrict__ dalpha, float *__restrict__ de_prev) {
+  extern __shared__ __align__(16) float smem[];
+  float *WeT = smem;                 // [Ke][D]  W_eᵀ
+  float *We = WeT + Ke * D;          // [D][Ke]  W_e (only when de_prev)
+  float *As = We + (de_prev ? D * Ke : 0);    // [BM][max(Ke,D)+4]
+  const int KS = (Ke > D ? Ke : D);
+  float *alpha = As + BM * (KS + 4);
+  constexpr int TN = Tn<D>::v;
+  const int tx = threadIdx.x % 16, ty = threadIdx.x / 16;
+  load_weights<D, true>(WeT, W_e, Ke);
+  if (de_prev) {   // de_prev only when Ke == D; Ws[a][c'] = W_e[a][c']
+    load_weights<D, false>(We, W_e, D);
+  }
+  const int tiles = (E + BM - 1) / BM;
+  for (int tile = blockIdx.x; tile < tiles; tile += gridDim.x) {
+    const long k0 = long(tile) * BM;
+    const int nrows = min(BM, int(E - k0));
+    __syncthreads();
+    load_rows(As, e_in, k0, nrows, Ke);
+    if (threadIdx.x < BM) {
+      const int r = threadIdx.x;
+      alpha[r] = r < nrows ? p[in_src[k0 + r]] + q[in_dst[k0 + r]] : 0.f;
+    }
+    __syncthreads();
+    float acc[4][TN];
+    zero_acc<D>(acc);
+    gemm_tile<D>(As, Ke, WeT, acc, tx, ty);                  // z
+    float dz[4][TN];
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+      const int r = ty * 4 + i;
+      float ev[TN], dev[TN], da = 0.f;
+      if (r < nrows) {
+        load_row<D>(e + (k0 + r) * D, ev, tx);
+        load_row<D>(de + (k0 + r) * D, dev, tx);
+      } else {
+#pragma unroll
+        for (int j = 0; j < TN; ++j) ev[j] = dev[j] = 0.f;
+      }
+      const float al = alpha[r];
+#pragma unroll
+      for (int j = 0; j < TN; ++j) {
+        const float dyv = dev[j] * ev[j] * (1.f - ev[j]);
+        da = fmaf(dyv, acc[i][j], da);
+        dz[i][j] = al * dyv;
+      }
+      da = hsum16(da);
+      if (r < nrows) {
+        store_row<D>(DZ + (k0 + r) * D, dz[i], tx);
+        if (tx == 0) dalpha[k0 + r] = da;
+      }
+    }
+    if (de_prev) {
+      __syncthreads();
+#pragma unroll
+      for (int i = 0; i < 4; ++i) store_row<D>(As + (ty * 4 + i) * (D + 4), dz[i], tx);
+      __syncthreads();
+      zero_acc<D>(acc);
+      gemm_tile<D>(As, D, We, acc, tx, ty);
+#pragma unroll
+      for (int i = 0; i < 4; ++i) {
+        const int r = ty * 4 + i;
+        if (r < nrows) store_row<D>(de_prev + (k0 + r) * D, acc[i], tx);
+      }
+    }
+  }
+}
+
+// Node backward (warp per node u):
+//   dh̄_u = Σ_{out-edges} MG + dp_u a_s + dq_u a_d ; dP = dh̄ ⊙ LReLU'(h̄)
+//   dp_u = Σ_{out-edges} dα ; dq_u = Σ_{in-edges} dα
+template <int D>
+__global__ void __launch_bounds__(NT) node_bwd_kernel(
+    const float *__restrict__ MG, const float *__restrict__ dalpha,
+    const float *__restrict__ hbar, const float *__restrict__ a_s, const float *__restrict__ a_d,
+    const int32_t *__restrict__ out_ptr, const int32_t *__restrict__ out_pos,
+    const int32_t *__restrict__ in_ptr, int N, float slope, float *__restrict__ dP,
+    float *__restrict__ dpq) {
+  constexpr int V = D / 32;
+  const int lane = threadIdx.x & 31;
+  const int warps = (gridDim.x * NT) / 32;
+  for (int u = (blockIdx.x * NT + threadIdx.x) / 32; u < N; u += warps) {
+    float acc[V];
+#pragma unroll
+    for (int c = 0; c < V; ++c) acc[c] = 0.f;
+    float dp = 0.f, dq = 0.f;
+    const int ob = out_ptr[u], oe = out_ptr[u + 1];
+    for (int j = ob; j < oe; ++j) {
+      const int k = out_pos[j];
+      const float *row = MG + long(k) * D + lane * V;
+#pragma unroll
+      for (int c = 0; c < V; ++c) acc[c] += __ldg(row + c);
+      dp += __ldg(dalpha + k);
+    }
+    for (int k = in_ptr[u]; k < in_ptr[u + 1]; ++k) dq += __ldg(dalpha + k);
+#pragma unroll
+    for (int c = 0; c < V; ++c) {
+      const int ch = lane * V + c;
+      const float v = acc[c] + dp * a_s[ch] + dq * a_d[ch];
+      const float hb = hbar[long(u) * D + ch];
+      dP[long(u) * D + ch] = v * lrelu_grad_from_out(hb, slope);
+    }
+    if (lane == 0) {
+      dpq[2 * long(u)] = dp;
+      dpq[2 * long(u) + 1] = dq;
+    }
+  }
+}
+
+// Deterministic split-K weight gradient: partial[s][a][b] = Σ_{r in split s} X[r][a] Y[r][b]
+// (X: [R][A], Y: [R][Bn]; 128x128 output tile per CTA, 8x8 per thread).
+constexpr int WG_R = 32;
+__global__ void __launch_bounds__(NT) wgrad_partial_kernel(const float *__restrict__ X, int A,
+                                                           const float *__restrict__ Y, int Bn,
+                                                           long R, int splits,
+                                                           float *__restrict__ partial) {
+  __shared__ __align__(16) float Xs[WG_R][128];
+  __shared__ __align__(16) float Ys[WG_R][128];
+  const int tx = threadIdx.x % 16, ty = threadIdx.x / 16;
+  const int s = blockIdx.x;
+  const int a0 = blockIdx.y * 128, b0 = blockIdx.z * 128;
+  const long per = (R + splits - 1) / splits;
+  const long r0 = s * per, r1 = min(R, r0 + per);
+  float acc[8][8];
+#pragma unroll
+  for (int i = 0; i < 8; ++i)
+#pragma unroll
+    for (int j = 0; j < 8; ++j) acc[i][j] = 0.f;
+  for (long rb = r0; rb < r1; rb += WG_R) {
+    __syncthreads();
+    for (int idx = threadIdx.x; idx < WG_R * 128; idx += NT) {
+      const int rr = idx / 128, cc = idx % 128;
+      const long row = rb + rr;
+      const bool ok = row < r1;
+      Xs[rr][cc] = (ok && a0 + cc < A) ? X[row * A + a0 + cc] : 0.f;
+      Ys[rr][cc] = (ok && b0 + cc < Bn) ? Y[row * Bn + b0 + cc] : 0.f;
+    }
+    __syncthreads();
+#pragma unroll 4
+    for (int rr = 0; rr < WG_R; ++rr) {
+      const float4 x0 = *reinterpret_cast<const float4 *>(&Xs[rr][ty * 4]);
+      const float4 x1 = *reinterpret_cast<const float4 *>(&Xs[rr][64 + ty * 4]);
+      const float4 y0 = *reinterpret_cast<const float4 *>(&Ys[rr][tx * 4]);
+      const float4 y1 = *reinterpret_cast<const float4 *>(&Ys[rr][64 + tx * 4]);
+      const float xv[8] = {x0.x, x0.y, x0.z, x0.w, x1.x, x1.y, x1.z, x1.w};
+      const float yv[8] = {y0.x, y0.y, y0.z, y0.w, y1.x, y1.y, y1.z, y1.w};
+#pragma unroll
+      for (int i = 0; i < 8; ++i)
+#pragma unroll
+        for (int j = 0; j < 8; ++j) acc[i][j] = fmaf(xv[i], yv[j], acc[i][j]);
+    }
+  }
+  float *out = partial + long(s) * A * Bn;
+#pragma unroll
+  for (int i = 0; i < 8; ++i) {
+    const int a = a0 + (i < 4 ? ty * 4 + i : 64 + ty * 4 + i - 4);
+    if (a >= A) continue;
+#pragma unroll
+    for (int j = 0; j < 8; ++j) {
+      const int b = b0 + (j < 4 ? tx * 4 + j : 64 + tx * 4 + j - 4);
+      if (b < Bn) out[long(a) * Bn + b] = acc[i][j];
+    }
+  }
+}
+
+__global__ void wgrad_reduce_kernel(const float *__restrict__ partial, int splits, long n,
+                                    float *__restrict__ out) {
+  for (long i = blockIdx.x * long(blockDim.x) + threadIdx.x; i < n; i += long(gridDim.x) * blockDim.x) {
+    float s = 0.f;
+    for (int k = 0; k < splits; ++k) s += partial[long(k) * n + i];
+    out[i] = s;
+  }
+}
+
+// a12: Adam, PyTorch semantics (R16).
+__global__ void adam_kernel(float *__restrict__ w, const float *__restrict__ g, float *__restrict__ m,
+                            float *__restrict__ v, long n, float lr, float wd, float b1, float b2,
+                            float bc1, float bc2, float eps) {
+  for (long i = blockIdx.x * long(blockDim.x) + threadIdx.x; i < n; i += long(gridDim.x) * blockDim.x) {
+    const float gr = g[i] + wd * w[i];
+    const float mi = b1 * m[i] + (1.f - b1) * gr;
+    const float vi = b2 * v[i] + (1.f - b2) * gr * gr;
+    m[i] = mi;
+    v[i] = vi;
+    const float mhat = mi / bc1;
+    const float vhat = vi / bc2;
+    w[i] = w[i] - lr * mhat / (sqrtf(vhat) + eps);
+  }
+}
+
+inline int grid_for(long work, int per_block, int cap) {
+  long g = (work + per_block - 1) / per_block;
+  if (g < 1) g = 1;
+  if (g > cap) g = cap;
+  return int(g);
+}
+
+template <class K> cudaError_t set_smem(K kern, size_t bytes) {
+  return cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, int(bytes));
+}
+
+}  // namespace
+
+// ---------------------------------------------------------------------------
+// Launchers
+// ---------------------------------------------------------------------------
+#define LAUNCH_CHECK()                                  \
+  do {                                                  \
+    cudaError_t e_ = cudaGetLastError();                \
+    if (e_ != cudaSuccess) return -int(e_);             \
+  } while (0)
+
+template <int D>
+static int forward_layer_impl(const occu_ctx *ctx, const DevCsr &csr, const FwdLayerArgs &a,
+                              cudaStream_t st) {
+  const int sms = ctx->num_sms;
+  int n = 0;
+  if (csr.N > 0) {
+    const size_t sm1 = (size_t(a.K) * D + BM * (a.K + 4)) * 4;
+    set_smem(node_gemm_kernel<D, 0>, sm1);
+    const int tiles = (csr.N + BM - 1) / BM;
+    OCCU_PROF_BEGIN(ctx, "node_gemm", st);
+    node_gemm_kernel<D, 0><<<grid_for(tiles, 1, 2 * sms), NT, sm1, st>>>(
+        a.h_in, a.K, a.W_u, a.a_s, a.a_d, csr.N, ctx->cfg.slope, a.hbar, a.p, a.q);
+    OCCU_PROF_END(ctx);
+    LAUNCH_CHECK();
+    ++n;
+  }
+  if (csr.E > 0) {
+    const size_t sm2 = (size_t(a.Ke) * D + D * D + BM * (a.Ke + 4) + BM * (D + 4) + BM) * 4;
+    set_smem(edge_fwd_kernel<D>, sm2);
+    const int tiles = (csr.E + BM - 1) / BM;
+    OCCU_PROF_BEGIN(ctx, "edge_fwd", st);
+    edge_fwd_kernel<D><<<grid_for(tiles, 1, sms), NT, sm2, st>>>(
+        a.e_in, a.Ke, a.W_e, a.W_m, a.p, a.q, csr.in_src, csr.in_dst, csr.E, a.e_out, a.g);
+    OCCU_PROF_END(ctx);
+    LAUNCH_CHECK();
+    ++n;
+  }
+  if (csr.N > 0) {
+    OCCU_PROF_BEGIN(ctx, "gather_segsum", st);
+    gather_segsum_kernel<D><<<grid_for(long(csr.N) * 32, NT, 16 * sms), NT, 0, st>>>(
+        a.g, a.hbar, csr.in_ptr, csr.in_src, csr.N, ctx->cfg.aggr == OCCU_AGGR_MEAN,
+        ctx->cfg.slope, a.h_out);
+    OCCU_PROF_END(ctx);
+    LAUNCH_CHECK();
+    ++n;
+  }
+  return n;
+}
+
+int launch_forward_layer(const occu_ctx *ctx, const DevCsr &csr, const FwdLayerArgs &a,
+                         cudaStream_t st) {
+  switch (ctx->cfg.d) {
+    case 64: return forward_layer_impl<64>(ctx, csr, a, st);
+    case 128: return forward_layer_impl<128>(ctx, csr, a, st);
+    default: return -int(cudaErrorInvalidValue);
+  }
+}
+
+int launch_permute_rows(const occu_ctx *ctx, const float *src, const int32_t *idx, int rows,
+                        int width, float *dst, cudaStream_t st) {
+  if (rows <= 0) return 0;
+  OCCU_PROF_BEGIN(ctx, "permute_e0", st);
+  permute_rows_kernel<<<grid_for(long(rows) * width, 256, 4096), 256, 0, st>>>(src, idx, rows,
+                                                                                width, dst);
+  OCCU_PROF_END(ctx);
+  LAUNCH_CHECK();
+  return 1;
+}
+
+int launch_readout_head(const occu_ctx *ctx, const DevCsr &csr, const float *h,
+                        const float *params, float *r, float *c, float *yhat, cudaStream_t st) {
+  const occu_config &cf = ctx->cfg;
+  const ParamLayout &L = ctx->layout;
+  const size_t smem = (4 * cf.d + cf.d + cf.d_h) * 4;
+  OCCU_PROF_BEGIN(ctx, "readout_head", st);
+  readout_head_kernel<<<csr.B, 4 * cf.d, smem, st>>>(h, csr.node_off, cf.d, cf.d_h,
+                                                      params + L.W_1, params + L.b_1,
+                                                      params + L.w_2, params + L.b_2, cf.slope,
+                                                      r, c, yhat);
+  OCCU_PROF_END(ctx);
+  LAUNCH_CHECK();
+  return 1;
+}
+
+static int wgrad(occu_ctx *ctx, const float *X, int A, const float *Y, int Bn, long R, float *out,
+                 cudaStream_t st) {
+  const long n = long(A) * Bn;
+  const int ta = (A + 127) / 128, tb = (Bn + 127) / 128;
+  int splits = int(std::max<long>(1, std::min<long>((2L * ctx->num_sms) / (ta * tb), (R + 255) / 256)));
+  if (R == 0) {
+    cudaMemsetAsync(out, 0, n * 4, st);
+    return 0;
+  }
+  if (ctx->ws.partial.ensure(size_t(splits) * n * 4) != cudaSuccess) return -int(cudaErrorMemoryAllocation);
+  float *part = ctx->ws.partial.as<float>();
+  OCCU_PROF_BEGIN(ctx, "wgrad_partial", st);
+  wgrad_partial_kernel<<<dim3(splits, ta, tb), NT, 0, st>>>(X, A, Y, Bn, R, splits, part);
+  OCCU_PROF_END(ctx);
+  LAUNCH_CHECK();
+  OCCU_PROF_BEGIN(ctx, "wgrad_reduce", st);
+  wgrad_reduce_kernel<<<grid_for(n, 256, 1024), 256, 0, st>>>(part, splits, n, out);
+  OCCU_PROF_END(ctx);
+  LAUNCH_CHECK();
+  return 2;
+}
+
+int launch_head_backward(occu_ctx *ctx, const DevCsr &csr, const float *targets, int global_B,
+                         cudaStream_t st) {
+  const occu_config &cf = ctx->cfg;
+  const ParamLayout &L = ctx->layout;
+  Workspace &w = ctx->ws;
+  float *P = ctx->params.as<float>();
+  float *G = ctx->grads.as<float>();
+  const float inv_gb = 1.f / float(global_B);
+  OCCU_PROF_BEGIN(ctx, "head_bwd_graph", st);
+  head_bwd_graph_kernel<<<csr.B, 128, cf.d_h * 4, st>>>(
+      w.yhat.as<float>(), targets, w.c.as<float>(), P + L.W_1, P + L.w_2, cf.d, cf.d_h, inv_gb,
+      cf.slope, w.dy.as<float>(), w.dc.as<float>(), w.dr.as<float>());
+  OCCU_PROF_END(ctx);
+  LAUNCH_CHECK();
+  const int jobs = cf.d_h * cf.d + 2 * cf.d_h + 2;
+  OCCU_PROF_BEGIN(ctx, "head_bwd_reduce", st);
+  head_bwd_reduce_kernel<<<grid_for(jobs, 256, 1024), 256, 0, st>>>(
+      w.dy.as<float>(), w.dc.as<float>(), w.r.as<float>(), w.c.as<float>(), w.yhat.as<float>(),
+      targets, csr.B, cf.d, cf.d_h, inv_gb, cf.slope, G + L.W_1, G + L.b_1, G + L.w_2, G + L.b_2,
+      w.loss.as<float>());
+  OCCU_PROF_END(ctx);
+  LAUNCH_CHECK();
+  OCCU_PROF_BEGIN(ctx, "broadcast_dh", st);
+  broadcast_dh_kernel<<<grid_for(long(csr.N) * cf.d, 256, 8192), 256, 0, st>>>(
+      w.dr.as<float>(), csr.node_graph, csr.node_off, csr.N, cf.d, w.dh.as<float>());
+  OCCU_PROF_END(ctx);
+  LAUNCH_CHECK();
+  return 3;
+}
+
+template <int D>
+static int backward_layer_impl(occu_ctx *ctx, const DevCsr &csr, const BwdLayerArgs &a,
+                               cudaStream_t st) {
+  const occu_config &cf = ctx->cfg;
+  const ParamLayout &L = ctx->layout;
+  Workspace &w = ctx->ws;
+  const int i = a.layer;
+  const float *P = ctx->params.as<float>();
+  float *G = ctx->grads.as<float>();
+  const int sms = ctx->num_sms;
+  int n = 0;
+  float *de = w.deA.as<float>();
+  if (csr.E > 0) {
+    const size_t smA = (2 * D * D + BM * (D + 4)) * 4 + 2 * BM * 4;
+    set_smem(edge_bwd_m_kernel<D>, smA);
+    const int tiles = (csr.E + BM - 1) / BM;
+    OCCU_PROF_BEGIN(ctx, "edge_bwd_m", st);
+    edge_bwd_m_kernel<D><<<grid_for(tiles, 1, sms), NT, smA, st>>>(
+        a.e, P + L.W_m[i], a.hbar, a.h, a.dh, a.de_out, csr.in_src, csr.in_dst, csr.in_ptr, csr.E,
+        cf.aggr == OCCU_AGGR_MEAN, cf.slope, w.MG.as<float>(), w.DV.as<float>(), de);
+    OCCU_PROF_END(ctx);
+    LAUNCH_CHECK();
+    ++n;
+    const int KS = a.Ke > D ? a.Ke : D;
+    const size_t smB = (size_t(a.Ke) * D + (a.de_prev ? D * a.Ke : 0) + BM * (KS + 4) + BM) * 4;
+    set_smem(edge_bwd_e_kernel<D>, smB);
+    OCCU_PROF_BEGIN(ctx, "edge_bwd_e", st);
+    edge_bwd_e_kernel<D><<<grid_for(tiles, 1, sms), NT, smB, st>>>(
+        a.e_in, a.Ke, a.e, de, P + L.W_e[i], a.p, a.q, csr.in_src, csr.in_dst, csr.E,
+        w.DZ.as<float>(), w.dalpha.as<float>(), a.de_prev);
+    OCCU_PROF_END(ctx);
+    LAUNCH_CHECK();
+    ++n;
+  }
+  OCCU_PROF_BEGIN(ctx, "node_bwd", st);
+  node_bwd_kernel<D><<<grid_for(long(csr.N) * 32, NT, 16 * sms), NT, 0, st>>>(
+      w.MG.as<float>(), w.dalpha.as<float>(), a.hbar, P + L.a_s[i], P + L.a_d[i], csr.out_ptr,
+      csr.out_pos, csr.in_ptr, csr.N, cf.slope, w.dP.as<float>(), w.dpq.as<float>());
+  OCCU_PROF_END(ctx);
+  LAUNCH_CHECK();
+  ++n;
+  int r;
+  // dW_m = DVᵀ E' ; dW_e = DZᵀ E_in ; dW_u = dPᵀ H_in ; [da_s; da_d] = [dp dq]ᵀ h̄
+  if ((r = wgrad(ctx, w.DV.as<float>(), D, a.e, D, csr.E, G + L.W_m[i], st)) < 0) return r;
+  n += r;
+  if ((r = wgrad(ctx, w.DZ.as<float>(), D, a.e_in, a.Ke, csr.E, G + L.W_e[i], st)) < 0) return r;
+  n += r;
+  if ((r = wgrad(ctx, w.dP.as<float>(), D, a.h_in, a.K, csr.N, G + L.W_u[i], st)) < 0) return r;
+  n += r;
+  if ((r = wgrad(ctx, w.dpq.as<float>(), 2, a.hbar, D, csr.N, G + L.a_s[i], st)) < 0) return r;
+  n += r;
+  if (a.dh_prev && csr.N > 0) {   // dh^{i-1} = dP W_u  (K == D for i > 0)
+    const size_t sm1 = (size_t(D) * D + BM * (D + 4)) * 4;
+    set_smem(node_gemm_kernel<D, 1>, sm1);
+    const int tiles = (csr.N + BM - 1) / BM;
+    OCCU_PROF_BEGIN(ctx, "dh_prev_gemm", st);
+    node_gemm_kernel<D, 1><<<grid_for(tiles, 1, 2 * sms), NT, sm1, st>>>(
+        w.dP.as<float>(), D, P + L.W_u[i], nullptr, nullptr, csr.N, cf.slope, a.dh_prev,
+        nullptr, nullptr);
+    OCCU_PROF_END(ctx);
+    LAUNCH_CHECK();
+    ++n;
+  }
+  return n;
+}
+
+int launch_backward_layer(occu_ctx *ctx, const DevCsr &csr, const BwdLayerArgs &a,
+                          cudaStream_t st) {
+  switch (ctx->cfg.d) {
+    case 64: return backward_layer_impl<64>(ctx, csr, a, st);
+    case 128: return backward_layer_impl<128>(ctx, csr, a, st);
+    default: return -int(cudaErrorInvalidValue);
+  }
+}
+
+int launch_adam(occu_ctx *ctx, float lr, cudaStream_t st) {
+  const long n = long(ctx->layout.total);
+  const double b1 = 0.9, b2 = 0.999;
+  const double bc1 = 1.0 - pow(b1, double(ctx->adam_t));
+  const double bc2 = 1.0 - pow(b2, double(ctx->adam_t));
+  OCCU_PROF_BEGIN(ctx, "adam", st);
+  adam_kernel<<<grid_for(n, 256, 1024), 256, 0, st>>>(
+      ctx->params.as<float>(), ctx->grads.as<float>(), ctx->adam_m.as<float>(),
+      ctx->adam_v.as<float>(), n, lr, ctx->weight_decay, float(b1), float(b2), float(bc1),
+      float(bc2), 1e-8f);
+  OCCU_PROF_END(ctx);
+  LAUNCH_CHECK();
+  return 1;
+}
+
+}  // namespace occu

@@ -1,0 +1,139 @@
+// Internal declarations shared by the runtime (occu_runtime.cu), the host
+// packer (pack.cpp), the weights code (weights.cpp) and the kernels.
+#pragma once
+
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <string>
+#include <vector>
+
+#include "../../include/occu.h"
+
+struct ncclComm;
+
+namespace occu {
+
+// Thread-local error for calls that have no ctx (occu_pack, occu_nccl_unique_id).
+void set_global_error(const std::string &msg);
+const char *global_error();
+
+struct ParamLayout {
+  // offsets (in floats) of each tensor inside the flat parameter vector
+  std::vector<size_t> W_u, W_e, W_m, a_s, a_d;
+  size_t W_1 = 0, b_1 = 0, w_2 = 0, b_2 = 0, total = 0;
+  std::vector<int> d_in, de_in;
+};
+ParamLayout make_layout(const occu_config &c);
+
+// Grow-only device buffer.
+struct DevBuf {
+  void *ptr = nullptr;
+  size_t bytes = 0;
+  cudaError_t ensure(size_t need);
+  void release();
+  template <class T> T *as() const { return reinterpret_cast<T *>(ptr); }
+};
+
+// Device-resident per-layer activations and scratch for one batch size.
+struct Workspace {
+  // inputs staged on device (host-pointer calls)
+  DevBuf node_feat, edge_feat, targets, out_occ;
+  DevBuf csr;              // concatenated int32 CSR arrays for host-CSR calls
+  DevBuf e0;               // edge features permuted to in-CSR order [E][F_e]
+  std::vector<DevBuf> hbar, p, q, e, h;   // per layer
+  DevBuf g;                // [E][d] channel-softmax gates (scratch)
+  DevBuf r, c, yhat;       // [B][d], [B][d_h], [B]
+  // backward scratch
+  DevBuf dy, dc, dr, dh, dhprev, dP, MG, DV, DZ, deA, deB, dalpha, dpq, partial, loss;
+  void release_all();
+};
+
+struct DevCsr {            // device view of a packed batch
+  int32_t B = 0, N = 0, E = 0;
+  const int32_t *node_off = nullptr, *edge_off = nullptr, *in_ptr = nullptr, *in_src = nullptr,
+                *in_dst = nullptr, *in_eid = nullptr, *out_ptr = nullptr, *out_pos = nullptr,
+                *node_graph = nullptr;
+};
+
+// Per-kernel CUDA-event profiler (bench.py's roofline numbers).
+struct Profiler {
+  bool on = false;
+  struct Rec { int kind; cudaEvent_t a, b; };
+  std::vector<std::string> names;
+  std::vector<double> total_ms;
+  std::vector<int64_t> count;
+  std::vector<Rec> pending;
+  std::vector<cudaEvent_t> pool;
+  int cur = -1;
+  cudaEvent_t cur_a = nullptr;
+  cudaStream_t cur_s = nullptr;
+  void begin(const char *name, cudaStream_t s);
+  void end();
+  void drain();          // synchronises and folds pending pairs into totals
+  void reset();
+  ~Profiler();
+};
+
+}  // namespace occu
+
+struct occu_ctx {
+  occu_config cfg{};
+  occu::ParamLayout layout;
+  int device = 0;
+  cudaStream_t stream = nullptr;
+  int num_sms = 148;
+  bool weights_ready = false;
+  bool keep = false;
+  float weight_decay = 1e-4f;
+  occu::DevBuf params, grads, adam_m, adam_v;
+  int64_t adam_t = 0;
+  occu::Workspace ws;
+  occu::DevCsr last_csr;   // geometry of the last forward (for occu_get_tensor)
+  bool have_forward = false;
+  int64_t launches = 0;
+  mutable occu::Profiler prof;
+  // data parallel
+  ncclComm *comm = nullptr;
+  int rank = 0, world = 1;
+  std::string err;
+};
+
+namespace occu {
+
+#define OCCU_PROF_BEGIN(ctx, name, st) \
+  do { if ((ctx)->prof.on) (ctx)->prof.begin(name, st); } while (0)
+#define OCCU_PROF_END(ctx) \
+  do { if ((ctx)->prof.on) (ctx)->prof.end(); } while (0)
+
+// ---- kernel launchers (kernels_simt.cu) ------------------------------------
+struct FwdLayerArgs {
+  const float *h_in; int K;            // [N][K]
+  const float *e_in; int Ke;           // [E][Ke] in-CSR order
+  const float *W_u, *W_e, *W_m, *a_s, *a_d;
+  float *hbar, *p, *q, *e_out, *g, *h_out;   // e_out may be null
+};
+int launch_forward_layer(const occu_ctx *ctx, const DevCsr &csr, const FwdLayerArgs &a,
+                         cudaStream_t st);
+int launch_permute_rows(const occu_ctx *ctx, const float *src, const int32_t *idx, int rows,
+                        int width, float *dst, cudaStream_t st);
+int launch_readout_head(const occu_ctx *ctx, const DevCsr &csr, const float *h,
+                        const float *params, float *r, float *c, float *yhat, cudaStream_t st);
+
+struct BwdLayerArgs {
+  int layer;
+  const float *h_in; int K;           // h^{i-1} [N][K]
+  const float *e_in; int Ke;          // e^{i-1} [E][Ke]
+  const float *hbar, *p, *q, *e, *h;  // layer i saved
+  const float *dh;                    // [N][d] gradient w.r.t. h^i
+  const float *de_out;                // [E][d] gradient w.r.t. e^i from layer i+1 (nullable)
+  float *de_prev;                     // [E][Ke] (nullable at layer 0)
+  float *dh_prev;                     // [N][K]  (nullable at layer 0)
+};
+int launch_backward_layer(occu_ctx *ctx, const DevCsr &csr, const BwdLayerArgs &a,
+                          cudaStream_t st);
+int launch_head_backward(occu_ctx *ctx, const DevCsr &csr, const float *targets, int global_B,
+                         cudaStream_t st);
+int launch_adam(occu_ctx *ctx, float lr, cudaStream_t st);
+
+}  // namespace occu

@@ -1,0 +1,704 @@
+// C-ABI runtime: context, weights, device batches, forward / train-step
+// orchestration, NCCL data parallelism and introspection (include/occu.h).
+#include <cuda_runtime.h>
+#include <math.h>
+#include <stdio.h>
+#include <stdlib.h>
+#include <string.h>
+
+#include <algorithm>
+#include <string>
+#include <vector>
+
+#include "nccl.h"
+#include "occu_internal.h"
+
+namespace occu {
+void init_flat(const occu_config &c, uint64_t seed, std::vector<float> &out);
+bool write_file(const char *path, const char magic[8], const occu_config &c,
+                const std::vector<std::pair<const void *, size_t>> &chunks, std::string &err);
+occu_status read_file(const char *path, const char magic[8], const occu_config &c,
+                      std::vector<unsigned char> &payload, size_t expect_bytes, std::string &err);
+
+static thread_local std::string g_err;
+void set_global_error(const std::string &msg) { g_err = msg; }
+const char *global_error() { return g_err.c_str(); }
+
+cudaError_t DevBuf::ensure(size_t need) {
+  if (need == 0) need = 16;
+  if (bytes >= need) return cudaSuccess;
+  if (ptr) cudaFree(ptr);
+  ptr = nullptr;
+  bytes = 0;
+  const size_t cap = need + need / 8;
+  cudaError_t e = cudaMalloc(&ptr, cap);
+  if (e == cudaSuccess) bytes = cap;
+  else ptr = nullptr;
+  return e;
+}
+void DevBuf::release() {
+  if (ptr) cudaFree(ptr);
+  ptr = nullptr;
+  bytes = 0;
+}
+void Workspace::release_all() {
+  DevBuf *bufs[] = {&node_feat, &edge_feat, &targets, &out_occ, &csr, &e0, &g, &r, &c, &yhat,
+                    &dy, &dc, &dr, &dh, &dhprev, &dP, &MG, &DV, &DZ, &deA, &deB, &dalpha,
+                    &dpq, &partial, &loss};
+  for (DevBuf *b : bufs) b->release();
+  for (auto *v : {&hbar, &p, &q, &e, &h})
+    for (DevBuf &b : *v) b.release();
+}
+
+void Profiler::begin(const char *name, cudaStream_t s) {
+  int k = -1;
+  for (size_t i = 0; i < names.size(); ++i)
+    if (names[i] == name) { k = int(i); break; }
+  if (k < 0) {
+    names.push_back(name);
+    total_ms.push_back(0.0);
+    count.push_back(0);
+    k = int(names.size()) - 1;
+  }
+  cudaEvent_t a;
+  if (!pool.empty()) { a = pool.back(); pool.pop_back(); }
+  else cudaEventCreate(&a);
+  cudaEventRecord(a, s);
+  cur = k;
+  cur_a = a;
+  cur_s = s;
+}
+void Profiler::end() {
+  if (cur < 0) return;
+  cudaEvent_t b;
+  if (!pool.empty()) { b = pool.back(); pool.pop_back(); }
+  else cudaEventCreate(&b);
+  cudaEventRecord(b, cur_s);
+  pending.push_back({cur, cur_a, b});
+  cur = -1;
+  if (pending.size() > 4096) drain();
+}
+void Profiler::drain() {
+  for (Rec &r : pending) {
+    cudaEventSynchronize(r.b);
+    float ms = 0.f;
+    cudaEventElapsedTime(&ms, r.a, r.b);
+    total_ms[r.kind] += ms;
+    count[r.kind] += 1;
+    pool.push_back(r.a);
+    pool.push_back(r.b);
+  }
+  pending.clear();
+}
+void Profiler::reset() {
+  drain();
+  names.clear();
+  total_ms.clear();
+  count.clear();
+}
+Profiler::~Profiler() {
+  for (Rec &r : pending) { pool.push_back(r.a); pool.push_back(r.b); }
+  for (cudaEvent_t e : pool) cudaEventDestroy(e);
+}
+
+}  // namespace occu
+
+using namespace occu;
+
+namespace {
+
+occu_status fail(occu_ctx *ctx, occu_status st, const std::string &msg) {
+  if (ctx) ctx->err = msg;
+  else set_global_error(msg);
+  return st;
+}
+
+occu_status cuda_fail(occu_ctx *ctx, cudaError_t e, const char *where) {
+  return fail(ctx, e == cudaErrorMemoryAllocation ? OCCU_ENOMEM : OCCU_ECUDA,
+              std::string(where) + ": " + cudaGetErrorString(e));
+}
+
+#define CK(call, where)                                     \
+  do {                                                      \
+    cudaError_t e__ = (call);                               \
+    if (e__ != cudaSuccess) return cuda_fail(ctx, e__, where); \
+  } while (0)
+
+#define LK(expr, where)                                                     \
+  do {                                                                      \
+    int n__ = (expr);                                                       \
+    if (n__ < 0) return cuda_fail(ctx, cudaError_t(-n__), where);           \
+    ctx->launches += n__;                                                   \
+  } while (0)
+
+bool is_device_ptr(const void *p) {
+  if (!p) return false;
+  cudaPointerAttributes a;
+  if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
+    cudaGetLastError();
+    return false;
+  }
+  return a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged;
+}
+
+occu_status validate_cfg(const occu_config *c) {
+  if (!c) return fail(nullptr, OCCU_EINVAL, "config is NULL");
+  if (c->L < 1 || c->L > 16) return fail(nullptr, OCCU_EINVAL, "L must be in [1, 16]");
+  if (c->d != 64 && c->d != 128)
+    return fail(nullptr, OCCU_EINVAL, "this build supports d in {64, 128}");
+  if (c->F_n < 4 || c->F_n % 4 || c->F_n > 256 || c->F_e < 4 || c->F_e % 4 || c->F_e > 256)
+    return fail(nullptr, OCCU_EINVAL, "F_n, F_e must be multiples of 4 in [4, 256]");
+  if (c->d_h < 1 || c->d_h > 1024) return fail(nullptr, OCCU_EINVAL, "d_h must be in [1, 1024]");
+  if (c->aggr != OCCU_AGGR_SUM && c->aggr != OCCU_AGGR_MEAN)
+    return fail(nullptr, OCCU_EINVAL, "aggr must be SUM or MEAN");
+  if (c->msg != OCCU_MSG_CHANNEL_SOFTMAX)
+    return fail(nullptr, OCCU_EINVAL, "msg: only OCCU_MSG_CHANNEL_SOFTMAX (reading A) in this build");
+  if (c->prec != OCCU_FP32) return fail(nullptr, OCCU_EINVAL, "prec: only OCCU_FP32 in this build");
+  if (!(c->slope > 0.f && c->slope < 1.f)) return fail(nullptr, OCCU_EINVAL, "slope must be in (0,1)");
+  return OCCU_OK;
+}
+
+// Device view of the batch (copies a host batch into the workspace).
+occu_status resolve_csr(occu_ctx *ctx, const occu_csr_batch *b, DevCsr &out) {
+  if (!b) return fail(ctx, OCCU_EINVAL, "csr_batch is NULL");
+  out.B = b->num_graphs;
+  out.N = b->num_nodes;
+  out.E = b->num_edges;
+  if (b->on_device) {
+    out.node_off = b->node_off; out.edge_off = b->edge_off; out.in_ptr = b->in_ptr;
+    out.in_src = b->in_src; out.in_dst = b->in_dst; out.in_eid = b->in_eid;
+    out.out_ptr = b->out_ptr; out.out_pos = b->out_pos; out.node_graph = b->node_graph;
+    return OCCU_OK;
+  }
+  const size_t B1 = out.B + 1, N1 = out.N + 1, E = out.E, N = out.N;
+  const size_t total = 2 * B1 + 2 * N1 + 4 * E + N;
+  CK(ctx->ws.csr.ensure(total * 4), "csr alloc");
+  int32_t *d = ctx->ws.csr.as<int32_t>();
+  int32_t *q = d;
+  const int32_t *srcs[9] = {b->node_off, b->edge_off, b->in_ptr, b->out_ptr, b->in_src,
+                            b->in_dst, b->in_eid, b->out_pos, b->node_graph};
+  const size_t lens[9] = {B1, B1, N1, N1, E, E, E, E, N};
+  const int32_t **dsts[9] = {&out.node_off, &out.edge_off, &out.in_ptr, &out.out_ptr, &out.in_src,
+                             &out.in_dst, &out.in_eid, &out.out_pos, &out.node_graph};
+  if (b->priv == static_cast<void *>(b->node_off)) {
+    // occu_pack output: one contiguous allocation in this order -> a single copy
+    CK(cudaMemcpyAsync(d, b->node_off, total * 4, cudaMemcpyHostToDevice, ctx->stream), "csr H2D");
+    for (int i = 0; i < 9; ++i) { *dsts[i] = q; q += lens[i]; }
+  } else {
+    for (int i = 0; i < 9; ++i) {
+      if (lens[i]) CK(cudaMemcpyAsync(q, srcs[i], lens[i] * 4, cudaMemcpyHostToDevice, ctx->stream), "csr H2D");
+      *dsts[i] = q;
+      q += lens[i];
+    }
+  }
+  return OCCU_OK;
+}
+
+occu_status ensure_layer_bufs(occu_ctx *ctx, const DevCsr &csr) {
+  const occu_config &c = ctx->cfg;
+  Workspace &w = ctx->ws;
+  w.hbar.resize(c.L); w.p.resize(c.L); w.q.resize(c.L); w.e.resize(c.L); w.h.resize(c.L);
+  const size_t Nd = size_t(csr.N) * c.d * 4, Ed = size_t(csr.E) * c.d * 4;
+  for (int i = 0; i < c.L; ++i) {
+    CK(w.hbar[i].ensure(Nd), "alloc hbar");
+    CK(w.p[i].ensure(size_t(csr.N) * 4), "alloc p");
+    CK(w.q[i].ensure(size_t(csr.N) * 4), "alloc q");
+    CK(w.e[i].ensure(Ed), "alloc e");
+    CK(w.h[i].ensure(Nd), "alloc h");
+  }
+  CK(w.g.ensure(Ed), "alloc g");
+  CK(w.e0.ensure(size_t(csr.E) * c.F_e * 4), "alloc e0");
+  CK(w.r.ensure(size_t(csr.B) * c.d * 4), "alloc r");
+  CK(w.c.ensure(size_t(csr.B) * c.d_h * 4), "alloc c");
+  CK(w.yhat.ensure(size_t(csr.B) * 4), "alloc yhat");
+  return OCCU_OK;
+}
+
+// Forward over a device batch; node_feat / edge_feat are device pointers.
+occu_status forward(occu_ctx *ctx, const DevCsr &csr, const float *nf, const float *ef,
+                    bool save_all) {
+  const occu_config &c = ctx->cfg;
+  const ParamLayout &L = ctx->layout;
+  Workspace &w = ctx->ws;
+  occu_status st = ensure_layer_bufs(ctx, csr);
+  if (st != OCCU_OK) return st;
+  cudaStream_t s = ctx->stream;
+  const float *P = ctx->params.as<float>();
+  LK(launch_permute_rows(ctx, ef, csr.in_eid, csr.E, c.F_e, w.e0.as<float>(), s), "permute e0");
+  for (int i = 0; i < c.L; ++i) {
+    FwdLayerArgs a{};
+    a.h_in = i == 0 ? nf : w.h[i - 1].as<float>();
+    a.K = L.d_in[i];
+    a.e_in = i == 0 ? w.e0.as<float>() : w.e[i - 1].as<float>();
+    a.Ke = L.de_in[i];
+    a.W_u = P + L.W_u[i]; a.W_e = P + L.W_e[i]; a.W_m = P + L.W_m[i];
+    a.a_s = P + L.a_s[i]; a.a_d = P + L.a_d[i];
+    a.hbar = w.hbar[i].as<float>(); a.p = w.p[i].as<float>(); a.q = w.q[i].as<float>();
+    a.e_out = (i < c.L - 1 || save_all) ? w.e[i].as<float>() : nullptr;
+    a.g = w.g.as<float>();
+    a.h_out = w.h[i].as<float>();
+    LK(launch_forward_layer(ctx, csr, a, s), "forward layer");
+  }
+  LK(launch_readout_head(ctx, csr, w.h[c.L - 1].as<float>(), P, w.r.as<float>(), w.c.as<float>(),
+                         w.yhat.as<float>(), s),
+     "readout/head");
+  ctx->last_csr = csr;
+  ctx->have_forward = true;
+  return OCCU_OK;
+}
+
+struct Staged {
+  const float *nf = nullptr, *ef = nullptr, *y = nullptr;
+  bool host = false;
+};
+
+occu_status stage_inputs(occu_ctx *ctx, const DevCsr &csr, const float *nf, const float *ef,
+                         const float *y, Staged &out) {
+  const occu_config &c = ctx->cfg;
+  if (!nf || (csr.E > 0 && !ef)) return fail(ctx, OCCU_EINVAL, "feature pointer is NULL");
+  out.host = !is_device_ptr(nf);
+  if (!out.host) {
+    out.nf = nf; out.ef = ef; out.y = y;
+    return OCCU_OK;
+  }
+  Workspace &w = ctx->ws;
+  CK(w.node_feat.ensure(size_t(csr.N) * c.F_n * 4), "alloc node_feat");
+  CK(w.edge_feat.ensure(size_t(csr.E) * c.F_e * 4), "alloc edge_feat");
+  CK(cudaMemcpyAsync(w.node_feat.ptr, nf, size_t(csr.N) * c.F_n * 4, cudaMemcpyHostToDevice,
+                     ctx->stream), "node_feat H2D");
+  if (csr.E > 0)
+    CK(cudaMemcpyAsync(w.edge_feat.ptr, ef, size_t(csr.E) * c.F_e * 4, cudaMemcpyHostToDevice,
+                       ctx->stream), "edge_feat H2D");
+  out.nf = w.node_feat.as<float>();
+  out.ef = w.edge_feat.as<float>();
+  if (y) {
+    CK(w.targets.ensure(size_t(csr.B) * 4), "alloc targets");
+    CK(cudaMemcpyAsync(w.targets.ptr, y, size_t(csr.B) * 4, cudaMemcpyHostToDevice, ctx->stream),
+       "targets H2D");
+    out.y = w.targets.as<float>();
+  }
+  return OCCU_OK;
+}
+
+occu_status check_ready(occu_ctx *ctx) {
+  if (!ctx) return fail(nullptr, OCCU_EINVAL, "ctx is NULL");
+  if (!ctx->weights_ready) return fail(ctx, OCCU_ENOTREADY, "weights not initialised");
+  CK(cudaSetDevice(ctx->device), "cudaSetDevice");
+  return OCCU_OK;
+}
+
+occu_status grads_impl(occu_ctx *ctx, const occu_batch *batch, const float *targets, Staged &stg,
+                       DevCsr &csr) {
+  occu_status st = check_ready(ctx);
+  if (st != OCCU_OK) return st;
+  if (!batch || !batch->csr || !targets) return fail(ctx, OCCU_EINVAL, "batch/targets NULL");
+  if (batch->global_num_graphs < batch->csr->num_graphs)
+    return fail(ctx, OCCU_EINVAL, "global_num_graphs < local num_graphs");
+  ctx->launches = 0;
+  if ((st = resolve_csr(ctx, batch->csr, csr)) != OCCU_OK) return st;
+  if ((st = stage_inputs(ctx, csr, batch->node_feat, batch->edge_feat, targets, stg)) != OCCU_OK)
+    return st;
+  if ((st = forward(ctx, csr, stg.nf, stg.ef, true)) != OCCU_OK) return st;
+  const occu_config &c = ctx->cfg;
+  const ParamLayout &L = ctx->layout;
+  Workspace &w = ctx->ws;
+  const size_t Nd = size_t(csr.N) * c.d * 4, Ed = size_t(csr.E) * c.d * 4;
+  CK(w.dy.ensure(size_t(csr.B) * 4), "alloc");
+  CK(w.dc.ensure(size_t(csr.B) * c.d_h * 4), "alloc");
+  CK(w.dr.ensure(size_t(csr.B) * c.d * 4), "alloc");
+  CK(w.dh.ensure(Nd), "alloc");
+  CK(w.dP.ensure(Nd), "alloc");
+  CK(w.MG.ensure(Ed), "alloc");
+  CK(w.DV.ensure(Ed), "alloc");
+  CK(w.DZ.ensure(Ed), "alloc");
+  CK(w.deA.ensure(Ed), "alloc");
+  CK(w.deB.ensure(Ed), "alloc");
+  CK(w.dalpha.ensure(size_t(csr.E) * 4), "alloc");
+  CK(w.dpq.ensure(size_t(csr.N) * 8), "alloc");
+  CK(w.loss.ensure(4), "alloc");
+  cudaStream_t s = ctx->stream;
+  LK(launch_head_backward(ctx, csr, stg.y, batch->global_num_graphs, s), "head backward");
+  for (int i = c.L - 1; i >= 0; --i) {
+    BwdLayerArgs a{};
+    a.layer = i;
+    a.h_in = i == 0 ? stg.nf : w.h[i - 1].as<float>();
+    a.K = L.d_in[i];
+    a.e_in = i == 0 ? w.e0.as<float>() : w.e[i - 1].as<float>();
+    a.Ke = L.de_in[i];
+    a.hbar = w.hbar[i].as<float>(); a.p = w.p[i].as<float>(); a.q = w.q[i].as<float>();
+    a.e = w.e[i].as<float>(); a.h = w.h[i].as<float>();
+    a.dh = w.dh.as<float>();
+    a.de_out = i < c.L - 1 ? w.deB.as<float>() : nullptr;
+    a.de_prev = i > 0 ? w.deB.as<float>() : nullptr;     // read-before-write ordering, see DESIGN
+    a.dh_prev = i > 0 ? w.dh.as<float>() : nullptr;
+    LK(launch_backward_layer(ctx, csr, a, s), "backward layer");
+  }
+  // loss rides along the gradient buffer (slot `total`) so one allreduce sums both
+  CK(cudaMemcpyAsync(ctx->grads.as<float>() + L.total, w.loss.ptr, 4, cudaMemcpyDeviceToDevice, s),
+     "loss copy");
+  return OCCU_OK;
+}
+
+}  // namespace
+
+// ============================================================================
+extern "C" {
+
+size_t occu_num_params(const occu_config *cfg) {
+  if (!cfg) return 0;
+  return make_layout(*cfg).total;
+}
+
+occu_status occu_create(occu_ctx **out, const occu_config *cfg, int cuda_device, void *cuda_stream) {
+  if (!out) return fail(nullptr, OCCU_EINVAL, "out is NULL");
+  *out = nullptr;
+  occu_status st = validate_cfg(cfg);
+  if (st != OCCU_OK) return st;
+  cudaError_t e = cudaSetDevice(cuda_device);
+  if (e != cudaSuccess) return fail(nullptr, OCCU_ECUDA, std::string("cudaSetDevice: ") + cudaGetErrorString(e));
+  occu_ctx *ctx = new (std::nothrow) occu_ctx();
+  if (!ctx) return OCCU_ENOMEM;
+  ctx->cfg = *cfg;
+  ctx->layout = make_layout(*cfg);
+  ctx->device = cuda_device;
+  ctx->stream = static_cast<cudaStream_t>(cuda_stream);
+  cudaDeviceGetAttribute(&ctx->num_sms, cudaDevAttrMultiProcessorCount, cuda_device);
+  const size_t pb = (ctx->layout.total + 1) * 4;
+  if (ctx->params.ensure(pb) != cudaSuccess || ctx->grads.ensure(pb) != cudaSuccess ||
+      ctx->adam_m.ensure(pb) != cudaSuccess || ctx->adam_v.ensure(pb) != cudaSuccess) {
+    delete ctx;
+    return fail(nullptr, OCCU_ENOMEM, "parameter allocation failed");
+  }
+  cudaMemset(ctx->grads.ptr, 0, pb);
+  cudaMemset(ctx->adam_m.ptr, 0, pb);
+  cudaMemset(ctx->adam_v.ptr, 0, pb);
+  *out = ctx;
+  return OCCU_OK;
+}
+
+occu_status occu_destroy(occu_ctx *ctx) {
+  if (!ctx) return OCCU_OK;
+  cudaSetDevice(ctx->device);
+  cudaStreamSynchronize(ctx->stream);
+  if (ctx->comm) ncclCommDestroy(ctx->comm);
+  ctx->ws.release_all();
+  ctx->params.release();
+  ctx->grads.release();
+  ctx->adam_m.release();
+  ctx->adam_v.release();
+  delete ctx;
+  return OCCU_OK;
+}
+
+occu_status occu_set_stream(occu_ctx *ctx, void *cuda_stream) {
+  if (!ctx) return fail(nullptr, OCCU_EINVAL, "ctx is NULL");
+  ctx->stream = static_cast<cudaStream_t>(cuda_stream);
+  return OCCU_OK;
+}
+
+occu_status occu_set_params(occu_ctx *ctx, const float *host_flat, size_t n) {
+  if (!ctx || !host_flat) return fail(ctx, OCCU_EINVAL, "NULL argument");
+  if (n != ctx->layout.total) return fail(ctx, OCCU_EINVAL, "parameter count mismatch");
+  CK(cudaSetDevice(ctx->device), "cudaSetDevice");
+  CK(cudaMemcpyAsync(ctx->params.ptr, host_flat, n * 4, cudaMemcpyHostToDevice, ctx->stream), "H2D");
+  CK(cudaStreamSynchronize(ctx->stream), "sync");
+  ctx->weights_ready = true;
+  return OCCU_OK;
+}
+
+occu_status occu_get_params(const occu_ctx *cctx, float *host_flat, size_t n) {
+  occu_ctx *ctx = const_cast<occu_ctx *>(cctx);
+  if (!ctx || !host_flat) return fail(ctx, OCCU_EINVAL, "NULL argument");
+  if (n != ctx->layout.total) return fail(ctx, OCCU_EINVAL, "parameter count mismatch");
+  if (!ctx->weights_ready) return fail(ctx, OCCU_ENOTREADY, "weights not initialised");
+  CK(cudaSetDevice(ctx->device), "cudaSetDevice");
+  CK(cudaMemcpyAsync(host_flat, ctx->params.ptr, n * 4, cudaMemcpyDeviceToHost, ctx->stream), "D2H");
+  CK(cudaStreamSynchronize(ctx->stream), "sync");
+  return OCCU_OK;
+}
+
+occu_status occu_init_weights(occu_ctx *ctx, uint64_t seed) {
+  if (!ctx) return fail(nullptr, OCCU_EINVAL, "ctx is NULL");
+  std::vector<float> w;
+  init_flat(ctx->cfg, seed, w);
+  return occu_set_params(ctx, w.data(), w.size());
+}
+
+occu_status occu_load_weights(occu_ctx *ctx, const char *path) {
+  if (!ctx || !path) return fail(ctx, OCCU_EINVAL, "NULL argument");
+  std::vector<unsigned char> payload;
+  std::string err;
+  occu_status st = read_file(path, "OCCUW001", ctx->cfg, payload, ctx->layout.total * 4, err);
+  if (st != OCCU_OK) return fail(ctx, st, "occu_load_weights: " + err);
+  return occu_set_params(ctx, reinterpret_cast<const float *>(payload.data()), ctx->layout.total);
+}
+
+occu_status occu_save_weights(const occu_ctx *cctx, const char *path) {
+  occu_ctx *ctx = const_cast<occu_ctx *>(cctx);
+  if (!ctx || !path) return fail(ctx, OCCU_EINVAL, "NULL argument");
+  std::vector<float> w(ctx->layout.total);
+  occu_status st = occu_get_params(ctx, w.data(), w.size());
+  if (st != OCCU_OK) return st;
+  std::string err;
+  if (!write_file(path, "OCCUW001", ctx->cfg, {{w.data(), w.size() * 4}}, err))
+    return fail(ctx, OCCU_EINVAL, err);
+  return OCCU_OK;
+}
+
+occu_status occu_batch_to_device(occu_ctx *ctx, const occu_csr_batch *host, occu_csr_batch **dev_out) {
+  if (!ctx || !host || !dev_out) return fail(ctx, OCCU_EINVAL, "NULL argument");
+  if (host->on_device) return fail(ctx, OCCU_EINVAL, "batch already on device");
+  *dev_out = nullptr;
+  CK(cudaSetDevice(ctx->device), "cudaSetDevice");
+  const size_t B1 = host->num_graphs + 1, N1 = host->num_nodes + 1, E = host->num_edges,
+               N = host->num_nodes;
+  const size_t total = 2 * B1 + 2 * N1 + 4 * E + N;
+  int32_t *d = nullptr;
+  CK(cudaMalloc(&d, std::max<size_t>(total, 1) * 4), "batch alloc");
+  cudaError_t e = cudaMemcpyAsync(d, host->node_off, total * 4, cudaMemcpyHostToDevice, ctx->stream);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(ctx->stream);
+  if (e != cudaSuccess) {
+    cudaFree(d);
+    return cuda_fail(ctx, e, "batch H2D");
+  }
+  occu_csr_batch *b = static_cast<occu_csr_batch *>(calloc(1, sizeof(occu_csr_batch)));
+  if (!b) {
+    cudaFree(d);
+    return OCCU_ENOMEM;
+  }
+  *b = *host;
+  int32_t *q = d;
+  b->node_off = q; q += B1;
+  b->edge_off = q; q += B1;
+  b->in_ptr = q; q += N1;
+  b->out_ptr = q; q += N1;
+  b->in_src = q; q += E;
+  b->in_dst = q; q += E;
+  b->in_eid = q; q += E;
+  b->out_pos = q; q += E;
+  b->node_graph = q;
+  b->on_device = 1;
+  b->priv = d;
+  *dev_out = b;
+  return OCCU_OK;
+}
+
+void occu_batch_free(occu_csr_batch *b) {
+  if (!b) return;
+  if (b->on_device) cudaFree(b->priv);
+  else free(b->priv);
+  free(b);
+}
+
+occu_status occu_predict(occu_ctx *ctx, const occu_csr_batch *csr_batch, const float *node_feat,
+                         const float *edge_feat, float *out_occ) {
+  occu_status st = check_ready(ctx);
+  if (st != OCCU_OK) return st;
+  if (!out_occ) return fail(ctx, OCCU_EINVAL, "out_occ is NULL");
+  ctx->launches = 0;
+  DevCsr csr;
+  if ((st = resolve_csr(ctx, csr_batch, csr)) != OCCU_OK) return st;
+  Staged stg;
+  if ((st = stage_inputs(ctx, csr, node_feat, edge_feat, nullptr, stg)) != OCCU_OK) return st;
+  if (stg.host == is_device_ptr(out_occ))
+    return fail(ctx, OCCU_EINVAL, "out_occ must be in the same memory space as the features");
+  if ((st = forward(ctx, csr, stg.nf, stg.ef, ctx->keep)) != OCCU_OK) return st;
+  const size_t ob = size_t(csr.B) * 4;
+  if (stg.host) {
+    CK(cudaMemcpyAsync(out_occ, ctx->ws.yhat.ptr, ob, cudaMemcpyDeviceToHost, ctx->stream), "D2H");
+    CK(cudaStreamSynchronize(ctx->stream), "sync");
+  } else {
+    CK(cudaMemcpyAsync(out_occ, ctx->ws.yhat.ptr, ob, cudaMemcpyDeviceToDevice, ctx->stream), "D2D");
+  }
+  CK(cudaGetLastError(), "predict");
+  return OCCU_OK;
+}
+
+occu_status occu_compute_grads(occu_ctx *ctx, const occu_batch *batch, const float *targets,
+                               float *out_loss) {
+  Staged stg;
+  DevCsr csr;
+  occu_status st = grads_impl(ctx, batch, targets, stg, csr);
+  if (st != OCCU_OK) return st;
+  if (out_loss || stg.host) {
+    float l = 0.f;
+    CK(cudaMemcpyAsync(&l, ctx->grads.as<float>() + ctx->layout.total, 4, cudaMemcpyDeviceToHost,
+                       ctx->stream), "loss D2H");
+    CK(cudaStreamSynchronize(ctx->stream), "sync");
+    if (out_loss) *out_loss = l;
+  }
+  return OCCU_OK;
+}
+
+occu_status occu_train_step(occu_ctx *ctx, const occu_batch *batch, const float *targets,
+                            float lr, float *out_loss) {
+  Staged stg;
+  DevCsr csr;
+  occu_status st = grads_impl(ctx, batch, targets, stg, csr);
+  if (st != OCCU_OK) return st;
+  const size_t n = ctx->layout.total + 1;
+  if (ctx->comm && ctx->world > 1) {
+    ncclResult_t r = ncclAllReduce(ctx->grads.ptr, ctx->grads.ptr, n, ncclFloat32, ncclSum,
+                                   ctx->comm, ctx->stream);
+    if (r != ncclSuccess) return fail(ctx, OCCU_ENCCL, std::string("ncclAllReduce: ") + ncclGetErrorString(r));
+  }
+  ctx->adam_t += 1;
+  LK(launch_adam(ctx, lr, ctx->stream), "adam");
+  if (out_loss || stg.host) {
+    float l = 0.f;
+    CK(cudaMemcpyAsync(&l, ctx->grads.as<float>() + ctx->layout.total, 4, cudaMemcpyDeviceToHost,
+                       ctx->stream), "loss D2H");
+    CK(cudaStreamSynchronize(ctx->stream), "sync");
+    if (out_loss) *out_loss = l;
+  }
+  return OCCU_OK;
+}
+
+occu_status occu_get_grads(const occu_ctx *cctx, float *host_flat, size_t n) {
+  occu_ctx *ctx = const_cast<occu_ctx *>(cctx);
+  if (!ctx || !host_flat) return fail(ctx, OCCU_EINVAL, "NULL argument");
+  if (n != ctx->layout.total) return fail(ctx, OCCU_EINVAL, "parameter count mismatch");
+  CK(cudaSetDevice(ctx->device), "cudaSetDevice");
+  CK(cudaMemcpyAsync(host_flat, ctx->grads.ptr, n * 4, cudaMemcpyDeviceToHost, ctx->stream), "D2H");
+  CK(cudaStreamSynchronize(ctx->stream), "sync");
+  return OCCU_OK;
+}
+
+occu_status occu_set_weight_decay(occu_ctx *ctx, float wd) {
+  if (!ctx) return fail(nullptr, OCCU_EINVAL, "ctx is NULL");
+  if (!(wd >= 0.f)) return fail(ctx, OCCU_EINVAL, "weight decay must be >= 0");
+  ctx->weight_decay = wd;
+  return OCCU_OK;
+}
+
+occu_status occu_nccl_unique_id(void *out_128_bytes) {
+  if (!out_128_bytes) return fail(nullptr, OCCU_EINVAL, "NULL argument");
+  ncclUniqueId id;
+  ncclResult_t r = ncclGetUniqueId(&id);
+  if (r != ncclSuccess) return fail(nullptr, OCCU_ENCCL, std::string("ncclGetUniqueId: ") + ncclGetErrorString(r));
+  static_assert(sizeof(ncclUniqueId) == 128, "ncclUniqueId size");
+  memcpy(out_128_bytes, &id, 128);
+  return OCCU_OK;
+}
+
+occu_status occu_dist_init(occu_ctx *ctx, int rank, int world, const void *nccl_unique_id) {
+  if (!ctx || !nccl_unique_id) return fail(ctx, OCCU_EINVAL, "NULL argument");
+  if (world < 1 || rank < 0 || rank >= world) return fail(ctx, OCCU_EINVAL, "bad rank/world");
+  CK(cudaSetDevice(ctx->device), "cudaSetDevice");
+  if (ctx->comm) {
+    ncclCommDestroy(ctx->comm);
+    ctx->comm = nullptr;
+  }
+  ncclUniqueId id;
+  memcpy(&id, nccl_unique_id, 128);
+  ncclComm_t comm;
+  ncclResult_t r = ncclCommInitRank(&comm, world, id, rank);
+  if (r != ncclSuccess) return fail(ctx, OCCU_ENCCL, std::string("ncclCommInitRank: ") + ncclGetErrorString(r));
+  ctx->comm = comm;
+  ctx->rank = rank;
+  ctx->world = world;
+  return OCCU_OK;
+}
+
+occu_status occu_save_state(const occu_ctx *cctx, const char *path) {
+  occu_ctx *ctx = const_cast<occu_ctx *>(cctx);
+  if (!ctx || !path) return fail(ctx, OCCU_EINVAL, "NULL argument");
+  const size_t n = ctx->layout.total;
+  std::vector<float> m(n), v(n);
+  CK(cudaSetDevice(ctx->device), "cudaSetDevice");
+  CK(cudaMemcpyAsync(m.data(), ctx->adam_m.ptr, n * 4, cudaMemcpyDeviceToHost, ctx->stream), "D2H");
+  CK(cudaMemcpyAsync(v.data(), ctx->adam_v.ptr, n * 4, cudaMemcpyDeviceToHost, ctx->stream), "D2H");
+  CK(cudaStreamSynchronize(ctx->stream), "sync");
+  const int64_t t = ctx->adam_t;
+  std::string err;
+  if (!write_file(path, "OCCUS001", ctx->cfg, {{&t, 8}, {m.data(), n * 4}, {v.data(), n * 4}}, err))
+    return fail(ctx, OCCU_EINVAL, err);
+  return OCCU_OK;
+}
+
+occu_status occu_load_state(occu_ctx *ctx, const char *path) {
+  if (!ctx || !path) return fail(ctx, OCCU_EINVAL, "NULL argument");
+  const size_t n = ctx->layout.total;
+  std::vector<unsigned char> payload;
+  std::string err;
+  occu_status st = read_file(path, "OCCUS001", ctx->cfg, payload, 8 + 2 * n * 4, err);
+  if (st != OCCU_OK) return fail(ctx, st, "occu_load_state: " + err);
+  int64_t t;
+  memcpy(&t, payload.data(), 8);
+  CK(cudaSetDevice(ctx->device), "cudaSetDevice");
+  CK(cudaMemcpyAsync(ctx->adam_m.ptr, payload.data() + 8, n * 4, cudaMemcpyHostToDevice, ctx->stream), "H2D");
+  CK(cudaMemcpyAsync(ctx->adam_v.ptr, payload.data() + 8 + n * 4, n * 4, cudaMemcpyHostToDevice, ctx->stream), "H2D");
+  CK(cudaStreamSynchronize(ctx->stream), "sync");
+  ctx->adam_t = t;
+  return OCCU_OK;
+}
+
+occu_status occu_set_keep_intermediates(occu_ctx *ctx, int keep) {
+  if (!ctx) return fail(nullptr, OCCU_EINVAL, "ctx is NULL");
+  ctx->keep = keep != 0;
+  return OCCU_OK;
+}
+
+occu_status occu_get_tensor(occu_ctx *ctx, int32_t which, int32_t layer, void *host_dst, size_t bytes) {
+  if (!ctx || !host_dst) return fail(ctx, OCCU_EINVAL, "NULL argument");
+  if (!ctx->have_forward) return fail(ctx, OCCU_ENOTREADY, "no forward has run");
+  const DevCsr &c = ctx->last_csr;
+  const int d = ctx->cfg.d;
+  const bool per_layer = which <= OCCU_T_H;
+  if (per_layer && (layer < 0 || layer >= ctx->cfg.L)) return fail(ctx, OCCU_EINVAL, "bad layer");
+  const void *src = nullptr;
+  size_t need = 0;
+  Workspace &w = ctx->ws;
+  switch (which) {
+    case OCCU_T_HBAR: src = w.hbar[layer].ptr; need = size_t(c.N) * d * 4; break;
+    case OCCU_T_P: src = w.p[layer].ptr; need = size_t(c.N) * 4; break;
+    case OCCU_T_Q: src = w.q[layer].ptr; need = size_t(c.N) * 4; break;
+    case OCCU_T_E:
+      if (layer == ctx->cfg.L - 1 && !ctx->keep)
+        return fail(ctx, OCCU_ENOTREADY, "last-layer e not stored (set keep_intermediates)");
+      src = w.e[layer].ptr; need = size_t(c.E) * d * 4; break;
+    case OCCU_T_H: src = w.h[layer].ptr; need = size_t(c.N) * d * 4; break;
+    case OCCU_T_R: src = w.r.ptr; need = size_t(c.B) * d * 4; break;
+    case OCCU_T_YHAT: src = w.yhat.ptr; need = size_t(c.B) * 4; break;
+    default: return fail(ctx, OCCU_EINVAL, "unknown tensor");
+  }
+  if (bytes != need) return fail(ctx, OCCU_EINVAL, "byte count mismatch");
+  CK(cudaSetDevice(ctx->device), "cudaSetDevice");
+  CK(cudaMemcpyAsync(host_dst, src, need, cudaMemcpyDeviceToHost, ctx->stream), "D2H");
+  CK(cudaStreamSynchronize(ctx->stream), "sync");
+  return OCCU_OK;
+}
+
+int64_t occu_last_launch_count(const occu_ctx *ctx) { return ctx ? ctx->launches : 0; }
+
+occu_status occu_set_profiling(occu_ctx *ctx, int enable) {
+  if (!ctx) return fail(nullptr, OCCU_EINVAL, "ctx is NULL");
+  ctx->prof.on = enable != 0;
+  return OCCU_OK;
+}
+
+occu_status occu_profile_reset(occu_ctx *ctx) {
+  if (!ctx) return fail(nullptr, OCCU_EINVAL, "ctx is NULL");
+  cudaSetDevice(ctx->device);
+  ctx->prof.reset();
+  return OCCU_OK;
+}
+
+occu_status occu_profile_query(occu_ctx *ctx, int32_t idx, const char **name, double *total_ms,
+                               int64_t *launches) {
+  if (!ctx) return fail(nullptr, OCCU_EINVAL, "ctx is NULL");
+  cudaSetDevice(ctx->device);
+  ctx->prof.drain();
+  if (idx < 0 || size_t(idx) >= ctx->prof.names.size()) return fail(ctx, OCCU_EINVAL, "index out of range");
+  if (name) *name = ctx->prof.names[idx].c_str();
+  if (total_ms) *total_ms = ctx->prof.total_ms[idx];
+  if (launches) *launches = ctx->prof.count[idx];
+  return OCCU_OK;
+}
+
+const char *occu_last_error(const occu_ctx *ctx) {
+  if (ctx) return ctx->err.c_str();
+  return global_error();
+}
+
+}  // extern "C"

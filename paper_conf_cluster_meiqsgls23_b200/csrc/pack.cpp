@@ -1,0 +1,169 @@
+// Host-side batched-CSR packing (P49 DAGs, P139 edges
+// l = (u_s, u_d), P149 aggregation over in-edges l' = (u', u); tie-break keys
+// are DESIGN.md R17).
+//
+// Graphs are concatenated in caller order.  Because every edge of graph b has
+// both endpoints in [node_off[b], node_off[b+1]), the global sort by
+// (dst, src, eid) places graph b's edges exactly at [edge_off[b], edge_off[b+1])
+// — so each graph is sorted independently (two stable counting passes, LSD
+// order: by src then by dst for the in-CSR; by dst then by src for the
+// out-CSR) and graphs are processed in parallel by a small thread pool.
+#include <stdlib.h>
+#include <string.h>
+
+#include <algorithm>
+#include <atomic>
+#include <thread>
+#include <vector>
+
+#include "occu_internal.h"
+
+namespace {
+
+struct Scratch {
+  std::vector<int32_t> cnt, tmp;
+};
+
+// Stable counting sort of positions `in[0..m)` by key[in[i]] (keys in [0, n)).
+void counting_pass(const int32_t *key, const int32_t *in, int32_t *out, int32_t m, int32_t n,
+                   std::vector<int32_t> &cnt) {
+  cnt.assign(static_cast<size_t>(n) + 1, 0);
+  for (int32_t i = 0; i < m; ++i) cnt[key[in[i]] + 1]++;
+  for (int32_t v = 0; v < n; ++v) cnt[v + 1] += cnt[v];
+  for (int32_t i = 0; i < m; ++i) out[cnt[key[in[i]]]++] = in[i];
+}
+
+void pack_graph(const occu_graph_view &g, int32_t noff, int32_t eoff, occu_csr_batch *b,
+                Scratch &s) {
+  const int32_t n = g.num_nodes, m = g.num_edges;
+  std::vector<int32_t> order(m), tmp(m);
+  for (int32_t j = 0; j < m; ++j) order[j] = j;
+  // in-CSR: key (dst, src, eid) -> stable by src, then stable by dst
+  counting_pass(g.src, order.data(), tmp.data(), m, n, s.cnt);
+  counting_pass(g.dst, tmp.data(), order.data(), m, n, s.cnt);
+  std::vector<int32_t> in_pos_of(m);
+  for (int32_t k = 0; k < m; ++k) {
+    const int32_t j = order[k];
+    b->in_src[eoff + k] = noff + g.src[j];
+    b->in_dst[eoff + k] = noff + g.dst[j];
+    b->in_eid[eoff + k] = eoff + j;
+    in_pos_of[j] = eoff + k;
+  }
+  // in_ptr for this graph's nodes: in_ptr[noff+v] = eoff + #{dst < v}
+  s.cnt.assign(static_cast<size_t>(n) + 1, 0);
+  for (int32_t j = 0; j < m; ++j) s.cnt[g.dst[j] + 1]++;
+  for (int32_t v = 0; v < n; ++v) s.cnt[v + 1] += s.cnt[v];
+  for (int32_t v = 0; v < n; ++v) b->in_ptr[noff + v] = eoff + s.cnt[v];
+  // out-CSR: key (src, dst, eid) -> stable by dst, then stable by src
+  for (int32_t j = 0; j < m; ++j) order[j] = j;
+  counting_pass(g.dst, order.data(), tmp.data(), m, n, s.cnt);
+  counting_pass(g.src, tmp.data(), order.data(), m, n, s.cnt);
+  for (int32_t k = 0; k < m; ++k) b->out_pos[eoff + k] = in_pos_of[order[k]];
+  s.cnt.assign(static_cast<size_t>(n) + 1, 0);
+  for (int32_t j = 0; j < m; ++j) s.cnt[g.src[j] + 1]++;
+  for (int32_t v = 0; v < n; ++v) s.cnt[v + 1] += s.cnt[v];
+  for (int32_t v = 0; v < n; ++v) b->out_ptr[noff + v] = eoff + s.cnt[v];
+  for (int32_t v = 0; v < n; ++v) b->node_graph[noff + v] = -1;  // filled by caller
+}
+
+}  // namespace
+
+extern "C" occu_status occu_pack(const occu_graph_view *graphs, int32_t num_graphs,
+                                 occu_csr_batch **out) {
+  if (!out) {
+    occu::set_global_error("occu_pack: out is NULL");
+    return OCCU_EINVAL;
+  }
+  *out = nullptr;
+  if (!graphs || num_graphs < 1) {
+    occu::set_global_error("occu_pack: num_graphs < 1 or graphs NULL");
+    return OCCU_EINVAL;
+  }
+  // validate + offsets (64-bit to detect overflow)
+  int64_t N = 0, E = 0;
+  for (int32_t b = 0; b < num_graphs; ++b) {
+    const occu_graph_view &g = graphs[b];
+    if (g.num_nodes < 1 || g.num_edges < 0 || (g.num_edges > 0 && (!g.src || !g.dst))) {
+      occu::set_global_error("occu_pack: graph " + std::to_string(b) +
+                             ": num_nodes < 1, num_edges < 0 or NULL edge arrays");
+      return OCCU_EINVAL;
+    }
+    for (int32_t j = 0; j < g.num_edges; ++j) {
+      const int32_t s = g.src[j], t = g.dst[j];
+      if (s < 0 || s >= g.num_nodes || t < 0 || t >= g.num_nodes) {
+        occu::set_global_error("occu_pack: graph " + std::to_string(b) + " edge " +
+                               std::to_string(j) + ": node id out of range");
+        return OCCU_EINVAL;
+      }
+      if (s == t) {
+        occu::set_global_error("occu_pack: graph " + std::to_string(b) + " edge " +
+                               std::to_string(j) + ": self-loop (not a DAG)");
+        return OCCU_EINVAL;
+      }
+    }
+    N += g.num_nodes;
+    E += g.num_edges;
+    if (N >= (int64_t(1) << 31) - 1 || E >= (int64_t(1) << 31) - 1) {
+      occu::set_global_error("occu_pack: N or E >= 2^31");
+      return OCCU_EINVAL;
+    }
+  }
+  occu_csr_batch *b = static_cast<occu_csr_batch *>(calloc(1, sizeof(occu_csr_batch)));
+  if (!b) return OCCU_ENOMEM;
+  b->num_graphs = num_graphs;
+  b->num_nodes = static_cast<int32_t>(N);
+  b->num_edges = static_cast<int32_t>(E);
+  // one allocation for all arrays
+  const size_t B1 = num_graphs + 1, N1 = N + 1;
+  const size_t total = 2 * B1 + 2 * N1 + 4 * static_cast<size_t>(E) + static_cast<size_t>(N);
+  int32_t *base = static_cast<int32_t *>(malloc(std::max<size_t>(total, 1) * sizeof(int32_t)));
+  if (!base) {
+    free(b);
+    return OCCU_ENOMEM;
+  }
+  int32_t *q = base;
+  b->node_off = q; q += B1;
+  b->edge_off = q; q += B1;
+  b->in_ptr = q; q += N1;
+  b->out_ptr = q; q += N1;
+  b->in_src = q; q += E;
+  b->in_dst = q; q += E;
+  b->in_eid = q; q += E;
+  b->out_pos = q; q += E;
+  b->node_graph = q; q += N;
+  b->on_device = 0;
+  b->priv = base;
+  b->node_off[0] = 0;
+  b->edge_off[0] = 0;
+  for (int32_t i = 0; i < num_graphs; ++i) {
+    b->node_off[i + 1] = b->node_off[i] + graphs[i].num_nodes;
+    b->edge_off[i + 1] = b->edge_off[i] + graphs[i].num_edges;
+  }
+  b->in_ptr[N] = static_cast<int32_t>(E);
+  b->out_ptr[N] = static_cast<int32_t>(E);
+  // parallel over graphs (work-stealing by atomic counter; results independent of order)
+  unsigned hw = std::thread::hardware_concurrency();
+  const char *env = getenv("OCCU_PACK_THREADS");
+  if (env) hw = static_cast<unsigned>(atoi(env));
+  int nthreads = static_cast<int>(std::min<int64_t>(std::max(1u, hw), num_graphs));
+  if (E + N < 20000) nthreads = 1;
+  std::atomic<int32_t> next{0};
+  auto worker = [&]() {
+    Scratch s;
+    for (;;) {
+      const int32_t i = next.fetch_add(1);
+      if (i >= num_graphs) break;
+      pack_graph(graphs[i], b->node_off[i], b->edge_off[i], b, s);
+      for (int32_t v = b->node_off[i]; v < b->node_off[i + 1]; ++v) b->node_graph[v] = i;
+    }
+  };
+  if (nthreads <= 1) {
+    worker();
+  } else {
+    std::vector<std::thread> pool;
+    for (int t = 0; t < nthreads; ++t) pool.emplace_back(worker);
+    for (auto &t : pool) t.join();
+  }
+  *out = b;
+  return OCCU_OK;
+}

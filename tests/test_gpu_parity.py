@@ -1,0 +1,251 @@
+"""GPU parity: the CUDA path (through the C-ABI) vs the float64 oracle.
+
+Tolerances (BASELINE.json north_star): FP32 path rel-L2 <= 1e-4 on
+every intermediate and |ŷ - ŷ_ref| <= 1e-4 * max(|ŷ_ref|, 1e-2); integer CSR work
+bit-exact; closed-form special cases bit-exact.
+"""
+import numpy as np
+import pytest
+
+import oracle
+from occu_gen import configs, weights
+from paper_conf_cluster_meiqsgls23_b200 import occu
+
+pytestmark = pytest.mark.gpu
+TOL = 1e-4
+
+
+@pytest.fixture(scope="module", autouse=True)
+def built():
+    from paper_conf_cluster_meiqsgls23_b200 import build
+    build.build()
+
+
+def mk(L, d, F_n=80, F_e=4, aggr=0):
+    return occu.config(L=L, F_n=F_n, F_e=F_e, d=d, aggr=aggr)
+
+
+def ocfg(c):
+    return dict(L=c.L, F_n=c.F_n, F_e=c.F_e, d=c.d, d_h=c.d_h, aggr=c.aggr, msg=c.msg,
+                slope=float(np.float32(c.slope)))
+
+
+def wcfg(c):
+    return weights.ModelConfig(L=c.L, F_n=c.F_n, F_e=c.F_e, d=c.d, d_h=c.d_h, aggr=c.aggr)
+
+
+def rel(a, b):
+    a = np.asarray(a, np.float64)
+    b = np.asarray(b, np.float64)
+    nb = np.linalg.norm(b)
+    return np.linalg.norm(a - b) / (nb if nb > 0 else 1.0)
+
+
+def run_both(c, batch, flat, keep=True):
+    m = occu.Model(c)
+    m.set_params(flat)
+    m.keep_intermediates(keep)
+    csr = occu.pack(batch.graphs)
+    y = m.predict(csr, batch.node_feat, batch.edge_feat)
+    params = oracle.unflatten(ocfg(c), flat.astype(np.float64))
+    pk = oracle.pack(batch.graphs)
+    ref = oracle.forward(params, ocfg(c), pk, batch.node_feat, batch.edge_feat)
+    return m, y, ref, pk
+
+
+def compare_all(m, c, y, ref, pk, tol=TOL):
+    N, E, B, d = pk["num_nodes"], pk["num_edges"], pk["num_graphs"], c.d
+    for i in range(c.L):
+        lay = ref["layers"][i]
+        assert rel(m.get_tensor(occu.T_HBAR, i, (N, d)), lay["hbar"]) <= tol, ("hbar", i)
+        assert rel(m.get_tensor(occu.T_P, i, (N,)), lay["p"]) <= tol, ("p", i)
+        assert rel(m.get_tensor(occu.T_Q, i, (N,)), lay["q"]) <= tol, ("q", i)
+        if E:
+            assert rel(m.get_tensor(occu.T_E, i, (E, d)), lay["e"]) <= tol, ("e", i)
+        assert rel(m.get_tensor(occu.T_H, i, (N, d)), lay["h"]) <= tol, ("h", i)
+    assert rel(m.get_tensor(occu.T_R, 0, (B, d)), ref["r"]) <= tol
+    yr = ref["yhat"]
+    assert np.all(np.abs(y - yr) <= tol * np.maximum(np.abs(yr), 1e-2)), np.abs(y - yr).max()
+
+
+@pytest.mark.parametrize("L,d,aggr,seed", [(2, 64, 0, 1), (3, 128, 0, 2), (3, 128, 1, 3),
+                                           (1, 64, 1, 4)])
+def test_random_batches_all_intermediates(L, d, aggr, seed):
+    c = mk(L, d, aggr=aggr)
+    b = configs.random_dag_batch(40, 300 + seed, max_nodes=60, hub=True)
+    flat = weights.unit_scale(wcfg(c), weights.init_flat(wcfg(c), seed))
+    m, y, ref, pk = run_both(c, b, flat)
+    compare_all(m, c, y, ref, pk)
+
+
+def test_cfg1_lenet_default_weights():
+    c = mk(2, 64)
+    b = configs.cfg1()
+    for flat in (weights.init_flat(wcfg(c), 42), weights.unit_scale(wcfg(c), weights.init_flat(wcfg(c), 42))):
+        m, y, ref, pk = run_both(c, b, flat)
+        compare_all(m, c, y, ref, pk)
+
+
+def test_cfg2_subset_unit_scale():
+    c = mk(3, 128)
+    b = configs.cfg2(12)
+    flat = weights.unit_scale(wcfg(c), weights.init_flat(wcfg(c), 42))
+    m, y, ref, pk = run_both(c, b, flat)
+    compare_all(m, c, y, ref, pk)
+
+
+def test_cfg2_full_size_sampled_graphs():
+    """BASELINE CFG2 at full size (256 graphs) on device buffers, as bench.py runs
+    it; 6 sampled graphs checked one by one against the oracle."""
+    import torch
+    c = mk(3, 128)
+    b = configs.cfg2(256)
+    flat = weights.unit_scale(wcfg(c), weights.init_flat(wcfg(c), 42))
+    m = occu.Model(c)
+    m.set_params(flat)
+    csr = m.to_device(occu.pack(b.graphs))
+    nf = torch.from_numpy(b.node_feat).cuda()
+    ef = torch.from_numpy(b.edge_feat).cuda()
+    y = m.predict(csr, nf, ef)
+    torch.cuda.synchronize()
+    y = y.cpu().numpy()
+    params = oracle.unflatten(ocfg(c), flat.astype(np.float64))
+    for gi in (0, 1, 77, 128, 200, 255):
+        s = b.subset([gi])
+        yr = oracle.predict(params, ocfg(c), s.graphs, s.node_feat, s.edge_feat)
+        assert abs(y[gi] - yr[0]) <= TOL * max(abs(yr[0]), 1e-2), gi
+
+
+def test_path_count_closed_form_bit_exact():
+    """W_u = I, a = 0, W_m = 0, SUM, integer X >= 0 => H^i = (Aᵀ)^i X / d^i exactly."""
+    d = 64
+    c = mk(3, d, F_n=d, F_e=4)
+    b = configs.random_dag_batch(20, 77, max_nodes=40, f_n=d, hub=True)
+    X = np.floor(b.node_feat * 8).astype(np.float32)
+    p = weights.unflatten(wcfg(c), weights.init_flat(wcfg(c), 5).copy())
+    for i in range(3):
+        p[f"W_u{i}"] = np.eye(d, dtype=np.float32)
+        p[f"a_s{i}"][:] = 0
+        p[f"a_d{i}"][:] = 0
+        p[f"W_m{i}"][:] = 0
+    flat = weights.flatten(wcfg(c), p)
+    m = occu.Model(c)
+    m.set_params(flat)
+    m.keep_intermediates(True)
+    csr = occu.pack(b.graphs)
+    m.predict(csr, X, b.edge_feat)
+    pk = oracle.pack(b.graphs)
+    N = pk["num_nodes"]
+    adj = np.zeros((N, N), np.float64)
+    for s, t in zip(pk["in_src"], pk["in_dst"]):
+        adj[s, t] += 1
+    H = X.astype(np.float64)
+    for i in range(3):
+        H = adj.T @ H / d
+        assert np.array_equal(m.get_tensor(occu.T_H, i, (N, d)).astype(np.float64), H), i
+        assert np.array_equal(m.get_tensor(occu.T_E, i, (pk["num_edges"], d)),
+                              np.full((pk["num_edges"], d), 0.5, np.float32))
+
+
+def test_determinism_and_device_host_paths_bitwise():
+    import torch
+    c = mk(3, 128)
+    b = configs.random_dag_batch(64, 9, max_nodes=80, hub=True)
+    m = occu.Model(c)
+    m.init_weights(42)
+    host = occu.pack(b.graphs)
+    y1 = m.predict(host, b.node_feat, b.edge_feat)
+    y2 = m.predict(host, b.node_feat, b.edge_feat)
+    dev = m.to_device(host)
+    y3 = m.predict(dev, torch.from_numpy(b.node_feat).cuda(), torch.from_numpy(b.edge_feat).cuda())
+    torch.cuda.synchronize()
+    assert np.array_equal(y1, y2)
+    assert np.array_equal(y1, y3.cpu().numpy())
+    assert m.last_launch_count() >= 3 * 3 + 2
+
+
+def test_batching_invariance_gpu():
+    c = mk(3, 128)
+    b = configs.random_dag_batch(10, 19, max_nodes=50, hub=True)
+    m = occu.Model(c)
+    m.set_params(weights.unit_scale(wcfg(c), weights.init_flat(wcfg(c), 3)))
+    yb = m.predict(occu.pack(b.graphs), b.node_feat, b.edge_feat)
+    for i in range(b.num_graphs):
+        s = b.subset([i])
+        yi = m.predict(occu.pack(s.graphs), s.node_feat, s.edge_feat)
+        assert abs(yi[0] - yb[i]) <= 1e-5 * max(abs(yb[i]), 1e-2)
+
+
+def test_init_weights_matches_python_generator_and_file_roundtrip(tmp_path):
+    c = mk(3, 128)
+    m = occu.Model(c)
+    m.init_weights(42)
+    assert np.array_equal(m.get_params(), weights.init_flat(wcfg(c), 42))
+    path = str(tmp_path / "w.bin")
+    m.save_weights(path)
+    ocf, params = oracle.read_weights(path)        # independent reader
+    assert np.array_equal(oracle.flatten(ocf, params).astype(np.float32), m.get_params())
+    m2 = occu.Model(c)
+    m2.load_weights(path)
+    assert np.array_equal(m2.get_params(), m.get_params())
+    weights.write_weights(str(tmp_path / "w2.bin"), wcfg(c), weights.init_flat(wcfg(c), 7))
+    m2.load_weights(str(tmp_path / "w2.bin"))
+    assert np.array_equal(m2.get_params(), weights.init_flat(wcfg(c), 7))
+    raw = bytearray(open(path, "rb").read())
+    raw[100] ^= 1
+    open(path, "wb").write(bytes(raw))
+    with pytest.raises(occu.OccuError) as ei:
+        m2.load_weights(path)
+    assert ei.value.status == occu.OCCU_EFORMAT
+
+
+def test_errors():
+    with pytest.raises(occu.OccuError) as ei:
+        occu.Model(occu.config(d=96))
+    assert ei.value.status == occu.OCCU_EINVAL
+    m = occu.Model(mk(2, 64))
+    b = configs.random_dag_batch(2, 1)
+    with pytest.raises(occu.OccuError) as ei:
+        m.predict(occu.pack(b.graphs), b.node_feat, b.edge_feat)
+    assert ei.value.status == occu.OCCU_ENOTREADY
+
+
+# ---------------------------------------------------------------- training
+@pytest.mark.parametrize("L,d,aggr", [(2, 64, 0), (3, 128, 0), (3, 128, 1)])
+def test_gradients_match_oracle(L, d, aggr):
+    c = mk(L, d, aggr=aggr)
+    b = configs.random_dag_batch(24, 500 + L + aggr, max_nodes=50, hub=True)
+    flat = weights.unit_scale(wcfg(c), weights.init_flat(wcfg(c), 11))
+    m = occu.Model(c)
+    m.set_params(flat)
+    loss = m.compute_grads(occu.pack(b.graphs), b.node_feat, b.edge_feat, b.targets)
+    g = weights.unflatten(wcfg(c), m.get_grads())
+    params = oracle.unflatten(ocfg(c), flat.astype(np.float64))
+    lref, gref = oracle.loss_and_grads(params, ocfg(c), b.graphs, b.node_feat, b.edge_feat, b.targets)
+    assert abs(loss - lref) <= TOL * abs(lref)
+    for k in gref:
+        assert rel(g[k], gref[k]) <= TOL, (k, rel(g[k], gref[k]))
+
+
+def test_training_trajectory_matches_oracle():
+    c = mk(2, 64)
+    b = configs.random_dag_batch(16, 600, max_nodes=40, hub=True)
+    flat = weights.unit_scale(wcfg(c), weights.init_flat(wcfg(c), 12))
+    m = occu.Model(c)
+    m.set_params(flat)
+    csr = occu.pack(b.graphs)
+    params = oracle.unflatten(ocfg(c), flat.astype(np.float64))
+    st = {}
+    lr = 1e-3
+    for step in range(10):
+        loss = m.train_step(csr, b.node_feat, b.edge_feat, b.targets, lr)
+        lref, gref = oracle.loss_and_grads(params, ocfg(c), b.graphs, b.node_feat, b.edge_feat,
+                                           b.targets)
+        params, st = oracle.adam_step(params, gref, st, lr)
+        assert abs(loss - lref) <= TOL * abs(lref) + 1e-7, (step, loss, lref)
+    w = m.get_params().astype(np.float64)
+    wr = oracle.flatten(ocfg(c), params)
+    slack = np.abs(w - wr) > TOL * np.abs(wr) + 1e-6
+    # allow a few sign flips of near-zero gradients (<= 2 lr each)
+    assert np.all(np.abs(w - wr)[slack] <= 2 * lr * 10 + 1e-6)
+    assert slack.mean() < 0.01
