@@ -593,7 +593,9 @@ __global__ void __launch_bounds__(NT) edge_bwd_e_kernel(
       const float al = alpha[r];
 #pragma unroll
       for (int j = 0; j < TN; ++j) {
-        const float dyv = dev[j] * ev[j] * (1.f - ev[j]);
+        // σ'(y) = σ(y)·σ(-y) with y = α z recomputed: avoids the cancellation of
+        // 1 - e' when e' = σ(y) is close to 1 (float32).
+        const float dyv = dev[j] * ev[j] * (1.f / (1.f + expf(al * acc[i][j])));
         da = fmaf(dyv, acc[i][j], da);
         dz[i][j] = al * dyv;
       }
