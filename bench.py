@@ -199,6 +199,7 @@ def main():
     ap.add_argument("--no-train", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--no-flush", action="store_true")
+    ap.add_argument("--path", type=int, default=0, help="0: tcgen05 3xTF32 (default), 1: SIMT FP32")
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3
@@ -227,6 +228,7 @@ def main():
     stream = torch.cuda.current_stream(dev)
     model = occu.Model(c, device=local, stream=stream.cuda_stream)
     model.init_weights(42)
+    model.set_kernel_path(args.path)
     batch = configs.cfg2(args.graphs)              # every rank: its own CFG2 shard (weak)
     B, N, E = batch.num_graphs, batch.num_nodes, batch.num_edges
     host_csr = occu.pack(batch.graphs)
@@ -377,7 +379,7 @@ def main():
             "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
             "config": {"workload": "CFG2 (BASELINE.json configs[1])", "graphs_per_rank": B,
                        "nodes_per_rank": N, "edges_per_rank": E, "L": 3, "d": 128, "F_n": 80,
-                       "F_e": 4, "precision": "fp32 (SIMT)",
+                       "F_e": 4, "precision": "fp32: tcgen05 3xTF32 split GEMMs, FP32 accumulate" if args.path == 0 else "fp32 (SIMT)",
                        "l2": "flushed between timed steps (256 MiB write)" if not args.no_flush else "not flushed",
                        "parallelism": f"graph-sharded x{world}, no collective"},
             "gpu_launches": launches,

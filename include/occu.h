@@ -169,6 +169,10 @@ typedef enum {
   OCCU_T_R = 5,      /* [B][d]  readout */
   OCCU_T_YHAT = 6    /* [B] */
 } occu_tensor;
+/* Forward kernel path: 0 (default) = tcgen05 tensor cores, 3xTF32 split
+ * products with FP32 accumulation in TMEM; 1 = CUDA-core FP32 (SIMT).  Both
+ * meet the FP32 tolerance; the backward currently runs on CUDA cores. */
+occu_status occu_set_kernel_path(occu_ctx *ctx, int path);
 /* Keep every intermediate of the next forward (costs memory/bandwidth). */
 occu_status occu_set_keep_intermediates(occu_ctx *ctx, int keep);
 /* Copy an intermediate of the last forward into host memory (float32; BF16

@@ -46,6 +46,7 @@ struct Workspace {
   DevBuf r, c, yhat;       // [B][d], [B][d_h], [B]
   // backward scratch
   DevBuf dy, dc, dr, dh, dhprev, dP, MG, DV, DZ, deA, deB, dalpha, dpq, partial, loss;
+  DevBuf tcpart;           // tensor-core aggregation: boundary-segment partials
   void release_all();
 };
 
@@ -85,6 +86,7 @@ struct occu_ctx {
   int num_sms = 148;
   bool weights_ready = false;
   bool keep = false;
+  int path = 0;            // 0: tensor cores (3xTF32), 1: CUDA-core SIMT FP32
   float weight_decay = 1e-4f;
   occu::DevBuf params, grads, adam_m, adam_v;
   int64_t adam_t = 0;
@@ -115,6 +117,10 @@ struct FwdLayerArgs {
 };
 int launch_forward_layer(const occu_ctx *ctx, const DevCsr &csr, const FwdLayerArgs &a,
                          cudaStream_t st);
+bool tc_supported(const occu_config &c);
+size_t tc_partial_floats(int E, int D);
+int launch_forward_layer_tc(const occu_ctx *ctx, const DevCsr &csr, const FwdLayerArgs &a,
+                            float *partial, cudaStream_t st);
 int launch_permute_rows(const occu_ctx *ctx, const float *src, const int32_t *idx, int rows,
                         int width, float *dst, cudaStream_t st);
 int launch_readout_head(const occu_ctx *ctx, const DevCsr &csr, const float *h,

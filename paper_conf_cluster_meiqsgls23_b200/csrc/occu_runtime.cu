@@ -44,7 +44,7 @@ void DevBuf::release() {
 void Workspace::release_all() {
   DevBuf *bufs[] = {&node_feat, &edge_feat, &targets, &out_occ, &csr, &e0, &g, &r, &c, &yhat,
                     &dy, &dc, &dr, &dh, &dhprev, &dP, &MG, &DV, &DZ, &deA, &deB, &dalpha,
-                    &dpq, &partial, &loss};
+                    &dpq, &partial, &loss, &tcpart};
   for (DevBuf *b : bufs) b->release();
   for (auto *v : {&hbar, &p, &q, &e, &h})
     for (DevBuf &b : *v) b.release();
@@ -237,7 +237,13 @@ occu_status forward(occu_ctx *ctx, const DevCsr &csr, const float *nf, const flo
     a.e_out = (i < c.L - 1 || save_all) ? w.e[i].as<float>() : nullptr;
     a.g = w.g.as<float>();
     a.h_out = w.h[i].as<float>();
-    LK(launch_forward_layer(ctx, csr, a, s), "forward layer");
+    if (ctx->path == 0 && tc_supported(c)) {
+      a.e_out = w.e[i].as<float>();            // the gate kernel re-reads e'
+      CK(w.tcpart.ensure(tc_partial_floats(csr.E, c.d) * 4), "alloc tc partials");
+      LK(launch_forward_layer_tc(ctx, csr, a, w.tcpart.as<float>(), s), "forward layer (tc)");
+    } else {
+      LK(launch_forward_layer(ctx, csr, a, s), "forward layer");
+    }
   }
   LK(launch_readout_head(ctx, csr, w.h[c.L - 1].as<float>(), P, w.r.as<float>(), w.c.as<float>(),
                          w.yhat.as<float>(), s),
@@ -630,6 +636,13 @@ occu_status occu_load_state(occu_ctx *ctx, const char *path) {
   CK(cudaMemcpyAsync(ctx->adam_v.ptr, payload.data() + 8 + n * 4, n * 4, cudaMemcpyHostToDevice, ctx->stream), "H2D");
   CK(cudaStreamSynchronize(ctx->stream), "sync");
   ctx->adam_t = t;
+  return OCCU_OK;
+}
+
+occu_status occu_set_kernel_path(occu_ctx *ctx, int path) {
+  if (!ctx) return fail(nullptr, OCCU_EINVAL, "ctx is NULL");
+  if (path != 0 && path != 1) return fail(ctx, OCCU_EINVAL, "path must be 0 (tensor cores) or 1 (SIMT)");
+  ctx->path = path;
   return OCCU_OK;
 }
 

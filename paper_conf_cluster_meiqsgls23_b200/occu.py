@@ -31,7 +31,7 @@ EXPORTS = [
     "occu_compute_grads", "occu_get_grads", "occu_set_weight_decay", "occu_nccl_unique_id",
     "occu_dist_init", "occu_save_state", "occu_load_state", "occu_set_keep_intermediates",
     "occu_get_tensor", "occu_last_launch_count", "occu_last_error", "occu_set_profiling",
-    "occu_profile_reset", "occu_profile_query",
+    "occu_profile_reset", "occu_profile_query", "occu_set_kernel_path",
 ]
 
 
@@ -105,6 +105,7 @@ def lib():
             "occu_last_launch_count": ([VP], C.c_int64),
             "occu_last_error": ([VP], C.c_char_p),
             "occu_set_profiling": ([VP, C.c_int], I32),
+            "occu_set_kernel_path": ([VP, C.c_int], I32),
             "occu_profile_reset": ([VP], I32),
             "occu_profile_query": ([VP, I32, P(C.c_char_p), P(C.c_double), P(C.c_int64)], I32),
         }
@@ -326,6 +327,10 @@ class Model:
     def dist_init(self, rank: int, world: int, uid: bytes):
         buf = (C.c_ubyte * 128).from_buffer_copy(uid)
         _check(lib().occu_dist_init(self._ctx, rank, world, buf), self._ctx)
+
+    def set_kernel_path(self, path: int):
+        """0 = tensor cores (3xTF32, default), 1 = CUDA-core SIMT FP32."""
+        _check(lib().occu_set_kernel_path(self._ctx, int(path)), self._ctx)
 
     # introspection
     def keep_intermediates(self, keep=True):

@@ -41,8 +41,9 @@ def rel(a, b):
     return np.linalg.norm(a - b) / (nb if nb > 0 else 1.0)
 
 
-def run_both(c, batch, flat, keep=True):
+def run_both(c, batch, flat, keep=True, path=0):
     m = occu.Model(c)
+    m.set_kernel_path(path)
     m.set_params(flat)
     m.keep_intermediates(keep)
     csr = occu.pack(batch.graphs)
@@ -68,14 +69,49 @@ def compare_all(m, c, y, ref, pk, tol=TOL):
     assert np.all(np.abs(y - yr) <= tol * np.maximum(np.abs(yr), 1e-2)), np.abs(y - yr).max()
 
 
+@pytest.mark.parametrize("path", [0, 1], ids=["tcgen05", "simt"])
 @pytest.mark.parametrize("L,d,aggr,seed", [(2, 64, 0, 1), (3, 128, 0, 2), (3, 128, 1, 3),
                                            (1, 64, 1, 4)])
-def test_random_batches_all_intermediates(L, d, aggr, seed):
+def test_random_batches_all_intermediates(L, d, aggr, seed, path):
     c = mk(L, d, aggr=aggr)
     b = configs.random_dag_batch(40, 300 + seed, max_nodes=60, hub=True)
     flat = weights.unit_scale(wcfg(c), weights.init_flat(wcfg(c), seed))
-    m, y, ref, pk = run_both(c, b, flat)
+    m, y, ref, pk = run_both(c, b, flat, path=path)
     compare_all(m, c, y, ref, pk)
+
+
+@pytest.mark.parametrize("path", [0, 1], ids=["tcgen05", "simt"])
+def test_hub_nodes_spanning_many_tiles(path):
+    """Destination segments longer than a 128-edge tile (hubs) and ragged tails."""
+    c = mk(2, 128)
+    graphs, nfs, efs = [], [], []
+    from occu_gen.prng import Rng
+    r = Rng(99)
+    for n, extra in ((400, 700), (3, 0), (300, 260), (1, 0), (130, 129)):
+        s = list(range(n - 1)) + list(r.randint(0, n - 2, extra))
+        t = list(range(1, n)) + [n - 1] * extra
+        graphs.append((n, np.array(s, np.int32), np.array(t, np.int32)))
+        nfs.append(r.uniform(n * 80).reshape(n, 80).astype(np.float32))
+        efs.append(r.uniform(len(s) * 4).reshape(len(s), 4).astype(np.float32))
+    b = configs.Batch(graphs, np.concatenate(nfs), np.concatenate(efs), np.zeros(len(graphs), np.float32),
+                      ["hub"] * len(graphs))
+    flat = weights.unit_scale(wcfg(c), weights.init_flat(wcfg(c), 8))
+    m, y, ref, pk = run_both(c, b, flat, path=path)
+    compare_all(m, c, y, ref, pk)
+
+
+def test_tc_and_simt_paths_agree():
+    c = mk(3, 128)
+    b = configs.cfg2(8)
+    m0 = occu.Model(c)
+    m0.init_weights(42)
+    m1 = occu.Model(c)
+    m1.init_weights(42)
+    m1.set_kernel_path(1)
+    csr = occu.pack(b.graphs)
+    y0 = m0.predict(csr, b.node_feat, b.edge_feat)
+    y1 = m1.predict(csr, b.node_feat, b.edge_feat)
+    assert np.all(np.abs(y0 - y1) <= 1e-5 * np.maximum(np.abs(y1), 1e-2))
 
 
 def test_cfg1_lenet_default_weights():
@@ -116,7 +152,8 @@ def test_cfg2_full_size_sampled_graphs():
         assert abs(y[gi] - yr[0]) <= TOL * max(abs(yr[0]), 1e-2), gi
 
 
-def test_path_count_closed_form_bit_exact():
+@pytest.mark.parametrize("path", [0, 1], ids=["tcgen05", "simt"])
+def test_path_count_closed_form_bit_exact(path):
     """W_u = I, a = 0, W_m = 0, SUM, integer X >= 0 => H^i = (Aᵀ)^i X / d^i exactly."""
     d = 64
     c = mk(3, d, F_n=d, F_e=4)
@@ -130,6 +167,7 @@ def test_path_count_closed_form_bit_exact():
         p[f"W_m{i}"][:] = 0
     flat = weights.flatten(wcfg(c), p)
     m = occu.Model(c)
+    m.set_kernel_path(path)
     m.set_params(flat)
     m.keep_intermediates(True)
     csr = occu.pack(b.graphs)
