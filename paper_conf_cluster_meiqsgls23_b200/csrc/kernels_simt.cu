@@ -804,6 +804,28 @@ static int forward_layer_impl(const occu_ctx *ctx, const DevCsr &csr, const FwdL
   return n;
 }
 
+template <int D>
+static int gather_impl(const occu_ctx *ctx, const DevCsr &csr, const float *g, const float *hbar,
+                       float *h_out, cudaStream_t st) {
+  if (csr.N <= 0) return 0;
+  OCCU_PROF_BEGIN(ctx, "gather_segsum", st);
+  gather_segsum_kernel<D><<<grid_for(long(csr.N) * 32, NT, 16 * ctx->num_sms), NT, 0, st>>>(
+      g, hbar, csr.in_ptr, csr.in_src, csr.N, ctx->cfg.aggr == OCCU_AGGR_MEAN, ctx->cfg.slope,
+      h_out);
+  OCCU_PROF_END(ctx);
+  LAUNCH_CHECK();
+  return 1;
+}
+
+int launch_gather_segsum(const occu_ctx *ctx, const DevCsr &csr, const float *g,
+                         const float *hbar, float *h_out, cudaStream_t st) {
+  switch (ctx->cfg.d) {
+    case 64: return gather_impl<64>(ctx, csr, g, hbar, h_out, st);
+    case 128: return gather_impl<128>(ctx, csr, g, hbar, h_out, st);
+    default: return -int(cudaErrorInvalidValue);
+  }
+}
+
 int launch_forward_layer(const occu_ctx *ctx, const DevCsr &csr, const FwdLayerArgs &a,
                          cudaStream_t st) {
   switch (ctx->cfg.d) {

@@ -121,6 +121,8 @@ bool tc_supported(const occu_config &c);
 size_t tc_partial_floats(int E, int D);
 int launch_forward_layer_tc(const occu_ctx *ctx, const DevCsr &csr, const FwdLayerArgs &a,
                             float *partial, cudaStream_t st);
+int launch_gather_segsum(const occu_ctx *ctx, const DevCsr &csr, const float *g,
+                         const float *hbar, float *h_out, cudaStream_t st);
 int launch_permute_rows(const occu_ctx *ctx, const float *src, const int32_t *idx, int rows,
                         int width, float *dst, cudaStream_t st);
 int launch_readout_head(const occu_ctx *ctx, const DevCsr &csr, const float *h,

@@ -58,7 +58,7 @@ __device__ __forceinline__ void fence_after_sync() {
 __host__ __device__ constexpr uint32_t idesc(uint32_t M, uint32_t N, uint32_t ab_format) {
   return (1u << 4) | (ab_format << 7) | (ab_format << 10) | ((N >> 3) << 17) | ((M >> 4) << 24);
 }
-constexpr uint32_t FMT_BF16 = 1, FMT_TF32 = 2;
+constexpr uint32_t FMT_F16 = 0, FMT_BF16 = 1, FMT_TF32 = 2;
 
 // Shared-memory matrix descriptor, K-major operand in the 128-byte-swizzle
 // canonical layout: 8-row x 128-byte atoms (16-byte chunk index XOR row%8),
@@ -82,7 +82,7 @@ __device__ __forceinline__ void mma_tf32_ts(uint32_t d_tmem, uint32_t a_tmem, ui
       "tcgen05.mma.cta_group::1.kind::tf32 [%0], [%1], %2, %3, p;\n\t}" ::"r"(d_tmem),
       "r"(a_tmem), "l"(b_desc), "r"(idsc), "r"(accumulate));
 }
-__device__ __forceinline__ void mma_bf16_ts(uint32_t d_tmem, uint32_t a_tmem, uint64_t b_desc,
+__device__ __forceinline__ void mma_f16_ts(uint32_t d_tmem, uint32_t a_tmem, uint64_t b_desc,
                                             uint32_t idsc, uint32_t accumulate) {
   asm volatile(
       "{\n\t.reg .pred p;\n\t"
@@ -90,6 +90,25 @@ __device__ __forceinline__ void mma_bf16_ts(uint32_t d_tmem, uint32_t a_tmem, ui
       "tcgen05.mma.cta_group::1.kind::f16 [%0], [%1], %2, %3, p;\n\t}" ::"r"(d_tmem),
       "r"(a_tmem), "l"(b_desc), "r"(idsc), "r"(accumulate));
 }
+// Plain arrive / arrive with an expected transaction byte count.
+__device__ __forceinline__ void mbar_arrive(uint64_t *bar) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t *bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)),
+               "r"(bytes)
+               : "memory");
+}
+// Bulk (non-tensor) async copy global -> shared, completing on an mbarrier.
+__device__ __forceinline__ void bulk_g2s(void *dst_smem, const void *src_gmem, uint32_t bytes,
+                                         uint64_t *bar) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+          smem_u32(dst_smem)),
+      "l"(src_gmem), "r"(bytes), "r"(smem_u32(bar))
+      : "memory");
+}
+
 // Arrive on an mbarrier when all previously issued MMAs of this thread complete.
 __device__ __forceinline__ void mma_commit(uint64_t *bar) {
   asm volatile(
@@ -137,6 +156,14 @@ __device__ __forceinline__ void split_tf32(float x, uint32_t &hi, uint32_t &lo) 
   asm("cvt.rna.tf32.f32 %0, %1;" : "=r"(h) : "f"(x));
   hi = h;
   lo = __float_as_uint(x - __uint_as_float(h));
+}
+
+// Byte offset of element (row, k) of a K-major fp16 operand stored as
+// [K/64 chunk][rows][128 B] SW128 atoms.
+__host__ __device__ inline uint32_t sw128_offset_f16(uint32_t row, uint32_t k, uint32_t rows) {
+  const uint32_t chunk = k >> 6, kin = k & 63;
+  const uint32_t unit = (kin >> 3) ^ (row & 7);
+  return chunk * rows * 128u + row * 128u + unit * 16u + (kin & 7) * 2u;
 }
 
 // Byte offset of element (row, k) of a K-major fp32 operand stored as

@@ -1,0 +1,33 @@
+"""Small driver for ncu: a few CFG2 forward (and optionally train) steps."""
+import argparse
+import os
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import torch  # noqa: E402
+
+from occu_gen import configs  # noqa: E402
+from paper_conf_cluster_meiqsgls23_b200 import occu  # noqa: E402
+
+ap = argparse.ArgumentParser()
+ap.add_argument("--steps", type=int, default=3)
+ap.add_argument("--path", type=int, default=0)
+ap.add_argument("--train", action="store_true")
+ap.add_argument("--graphs", type=int, default=256)
+a = ap.parse_args()
+dev = torch.device("cuda", 0)
+m = occu.Model(occu.config(L=3, F_n=80, F_e=4, d=128))
+m.init_weights(42)
+m.set_kernel_path(a.path)
+b = configs.cfg2(a.graphs)
+csr = m.to_device(occu.pack(b.graphs))
+nf = torch.from_numpy(b.node_feat).to(dev)
+ef = torch.from_numpy(b.edge_feat).to(dev)
+yt = torch.from_numpy(b.targets).to(dev)
+for _ in range(a.steps):
+    if a.train:
+        m.train_step(csr, nf, ef, yt, 1e-4, want_loss=False)
+    else:
+        m.predict(csr, nf, ef)
+torch.cuda.synchronize()
+print("done")
