@@ -40,7 +40,7 @@ namespace occu {
 namespace {
 
 constexpr int TM = 128;
-constexpr int NTH = 192;
+constexpr int NTH = 320;
 constexpr uint32_t TMEM_COLS = 512;
 constexpr int EPI_NODE = 0, EPI_EDGE = 1, EPI_GATE = 2;
 
@@ -65,7 +65,7 @@ struct Smem {
   float *slot0;
   int slot_floats;
   __device__ __forceinline__ float *slot(int j) const { return slot0 + j * slot_floats; }
-  uint64_t *full, *empty, *afull, *afree, *accfull, *accfree;
+  uint64_t *full, *empty, *afull, *accfull;
   uint32_t *tmem_slot;
   int *fexp;
   float *red;
@@ -93,9 +93,7 @@ __device__ __forceinline__ Smem carve(uint8_t *raw, int D, int K) {
   s.full = bars;
   s.empty = bars + 2;
   s.afull = bars + 4;
-  s.afree = bars + 6;
   s.accfull = bars + 8;
-  s.accfree = bars + 10;
   s.tmem_slot = reinterpret_cast<uint32_t *>(bars + 12);
   s.fexp = reinterpret_cast<int *>(bars + 12) + 4;
   s.red = reinterpret_cast<float *>(bars + 12) + 16;
@@ -162,9 +160,7 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(RowGemmArgs a) {
       tc::mbar_init(s.full + j, 1);
       tc::mbar_init(s.empty + j, 128);
       tc::mbar_init(s.afull + j, 128);
-      tc::mbar_init(s.afree + j, 1);
       tc::mbar_init(s.accfull + j, 1);
-      tc::mbar_init(s.accfree + j, 128);
     }
     tc::fence_mbar_init();
   }
@@ -180,7 +176,7 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(RowGemmArgs a) {
   const int my = blockIdx.x < tiles ? (tiles - 1 - int(blockIdx.x)) / int(gridDim.x) + 1 : 0;
 
   if (warp == 0) {
-    // ---------------- producer ----------------
+    // ---------------- producer: tile i -> slot i%2 ----------------
     for (int i = 0; i < my; ++i) {
       const int j = i & 1;
       const long r0 = long(blockIdx.x + i * gridDim.x) * TM;
@@ -192,14 +188,13 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(RowGemmArgs a) {
         tc::bulk_g2s(s.slot(j) + r * S, a.A + (r0 + r) * K, uint32_t(K) * 4, s.full + j);
     }
   } else if (warp == 1) {
-    // ---------------- MMA issuer ----------------
+    // ---------------- MMA issuer: tiles in order, A[i%2] -> ACC[i%2] ----------------
     const uint32_t idsc = tc::idesc(128, uint32_t(D), tc::FMT_F16);
     const uint32_t w0a = tc::smem_u32(s.w0), w1a = tc::smem_u32(s.w1);
     const int nk = (K + 15) / 16;
     for (int i = 0; i < my; ++i) {
       const int j = i & 1;
       tc::mbar_wait(s.afull + j, (i >> 1) & 1);
-      if (i >= 2) tc::mbar_wait(s.accfree + j, ((i >> 1) - 1) & 1);
       tc::fence_after_sync();
       if (lane == 0) {
         const uint32_t d = tmem + acc_col(j);
@@ -213,130 +208,121 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(RowGemmArgs a) {
           tc::mma_f16_ts(d, a1, b0, idsc, 1u);
         }
         tc::mma_commit(s.accfull + j);
-        tc::mma_commit(s.afree + j);
       }
       __syncwarp();
     }
   } else {
-    // ---------------- workers: thread = row ----------------
-    const int q = warp & 3;
-    const int row = q * 32 + lane;
-    const uint32_t lane_base = tmem + (uint32_t(q * 32) << 16);
-    int e_prev = 0;
-    float aux_prev = 0.f;
-    long r0_prev = 0;
-    int nrows_prev = 0;
-    for (int i = 0; i <= my; ++i) {
-      int e_cur = 0;
-      float aux_cur = 0.f;
-      long r0 = 0;
-      int nrows = 0;
-      if (i < my) {
-        const int j = i & 1;
-        r0 = long(blockIdx.x + i * gridDim.x) * TM;
-        nrows = min(TM, int(a.R - r0));
-        const bool live = row < nrows;
-        if (EPI == EPI_EDGE && live)
-          aux_cur = __ldg(a.pin + a.src[r0 + row]) + __ldg(a.qin + a.dst[r0 + row]);   // α (R1)
-        tc::mbar_wait(s.full + j, (i >> 1) & 1);
-        if (i >= 2) tc::mbar_wait(s.afree + j, ((i >> 1) - 1) & 1);
-        const float *rp = s.slot(j) + row * S;
-        float mx = 0.f;
-        if (live)
-          for (int k = 0; k < K; k += 4) {
-            const float4 v = *reinterpret_cast<const float4 *>(rp + k);
-            mx = fmaxf(mx, fmaxf(fmaxf(fabsf(v.x), fabsf(v.y)), fmaxf(fabsf(v.z), fabsf(v.w))));
-          }
-        e_cur = scale_exp(mx);
-        const float xs = ldexpf(1.f, e_cur);
-        for (int c0 = 0; c0 < Kpad / 2; c0 += 32) {
-          uint32_t x0[32], x1[32];
-#pragma unroll
-          for (int u = 0; u < 32; u += 2) {
-            const int k = 2 * (c0 + u);
-            float4 v = make_float4(0.f, 0.f, 0.f, 0.f);
-            if (live && k < K) v = *reinterpret_cast<const float4 *>(rp + k);
-            split2(v.x * xs, v.y * xs, x0[u], x1[u]);
-            split2(v.z * xs, v.w * xs, x0[u + 1], x1[u + 1]);
-          }
-          tc::tmem_st32(lane_base + a_col(j) + c0, x0);
-          tc::tmem_st32(lane_base + a_col(j) + Kpad / 2 + c0, x1);
+    // ---------------- workers: two ping-pong warpgroups (warps 2-5, 6-9) -------------
+    // group g handles local tiles i = g, g+2, ... : convert -> MMA -> epilogue, thread = row.
+    const int g = (warp - 2) >> 2;
+    const int qd = warp & 3;                       // TMEM lane quarter of this warp
+    const int row = qd * 32 + lane;
+    const uint32_t lane_base = tmem + (uint32_t(qd * 32) << 16);
+    for (int i = g; i < my; i += 2) {
+      const int j = i & 1;                         // == g
+      const uint32_t par = (i >> 1) & 1;
+      const long r0 = long(blockIdx.x + i * gridDim.x) * TM;
+      const int nrows = min(TM, int(a.R - r0));
+      const bool live = row < nrows;
+      float aux = 0.f;
+      if (EPI == EPI_EDGE && live)
+        aux = __ldg(a.pin + a.src[r0 + row]) + __ldg(a.qin + a.dst[r0 + row]);   // α (R1)
+      // -- convert the row into TMEM A[j] (its previous MMA finished: we consumed ACC[j])
+      tc::mbar_wait(s.full + j, par);
+      const float *rp = s.slot(j) + row * S;
+      float mx = 0.f;
+      if (live)
+#pragma unroll 8
+        for (int k = 0; k < K; k += 4) {
+          const float4 v = *reinterpret_cast<const float4 *>(rp + k);
+          mx = fmaxf(mx, fmaxf(fmaxf(fabsf(v.x), fabsf(v.y)), fmaxf(fabsf(v.z), fabsf(v.w))));
         }
-        tc::tmem_st_wait();
-        tc::fence_before_sync();
-        tc::mbar_arrive(s.empty + j);
-        tc::mbar_arrive(s.afull + j);
+      const int er = scale_exp(mx);
+      const float xs = ldexpf(1.f, er);
+      for (int c0 = 0; c0 < Kpad / 2; c0 += 32) {
+        uint32_t x0[32], x1[32];
+#pragma unroll
+        for (int u = 0; u < 32; u += 2) {
+          const int k = 2 * (c0 + u);
+          float4 v = make_float4(0.f, 0.f, 0.f, 0.f);
+          if (live && k < K) v = *reinterpret_cast<const float4 *>(rp + k);
+          split2(v.x * xs, v.y * xs, x0[u], x1[u]);
+          split2(v.z * xs, v.w * xs, x0[u + 1], x1[u + 1]);
+        }
+        tc::tmem_st32(lane_base + a_col(j) + c0, x0);
+        tc::tmem_st32(lane_base + a_col(j) + Kpad / 2 + c0, x1);
       }
-      if (i >= 1) {
-        // ---- epilogue of the previous tile ----
-        const int ip = i - 1, jp = ip & 1;
-        tc::mbar_wait(s.accfull + jp, (ip >> 1) & 1);
-        tc::fence_after_sync();
-        const float un = ldexpf(1.f, -(e_prev + fexp));
-        const bool live = row < nrows_prev;
-        const long grow = r0_prev + row;
-        float *orow = a.out + grow * D;
-        if (EPI == EPI_GATE) {
-          float v[D];
+      tc::tmem_st_wait();
+      tc::fence_before_sync();
+      tc::mbar_arrive(s.empty + j);
+      tc::mbar_arrive(s.afull + j);
+      // -- epilogue
+      tc::mbar_wait(s.accfull + j, par);
+      tc::fence_after_sync();
+      const float un = ldexpf(1.f, -(er + fexp));
+      const long grow = r0 + row;
+      float *orow = a.out + grow * D;
+      if (EPI == EPI_GATE) {
+        float v[D];
 #pragma unroll
-          for (int c0 = 0; c0 < D; c0 += 32) {
-            uint32_t r[32];
-            tc::tmem_ld32(lane_base + acc_col(jp) + c0, r);
-            tc::tmem_ld_wait();
+        for (int c0 = 0; c0 < D; c0 += 32) {
+          uint32_t r[32];
+          tc::tmem_ld32(lane_base + acc_col(j) + c0, r);
+          tc::tmem_ld_wait();
 #pragma unroll
-            for (int u = 0; u < 32; ++u) v[c0 + u] = __uint_as_float(r[u]) * un;
-          }
-          float m = -INFINITY;
+          for (int u = 0; u < 32; ++u) v[c0 + u] = __uint_as_float(r[u]) * un;
+        }
+        float m = -INFINITY;
 #pragma unroll
-          for (int c = 0; c < D; ++c) m = fmaxf(m, v[c]);
-          float sum = 0.f;
+        for (int c = 0; c < D; ++c) m = fmaxf(m, v[c]);
+        float sum = 0.f;
 #pragma unroll
-          for (int c = 0; c < D; ++c) {
-            v[c] = expf(v[c] - m);
-            sum += v[c];
-          }
-          if (live) {
+        for (int c = 0; c < D; ++c) {
+          v[c] = expf(v[c] - m);
+          sum += v[c];
+        }
+        const float inv = __frcp_rn(sum);
+        if (live) {
 #pragma unroll
-            for (int c = 0; c < D; c += 4)
-              *reinterpret_cast<float4 *>(orow + c) =
-                  make_float4(v[c] / sum, v[c + 1] / sum, v[c + 2] / sum, v[c + 3] / sum);
-          }
-        } else {
-          float pp = 0.f, qq = 0.f;
+          for (int c = 0; c < D; c += 4)
+            *reinterpret_cast<float4 *>(orow + c) =
+                make_float4(v[c] * inv, v[c + 1] * inv, v[c + 2] * inv, v[c + 3] * inv);
+        }
+      } else {
+        float pp = 0.f, qq = 0.f;
 #pragma unroll
-          for (int c0 = 0; c0 < D; c0 += 32) {
-            uint32_t r[32];
-            tc::tmem_ld32(lane_base + acc_col(jp) + c0, r);
-            tc::tmem_ld_wait();
+        for (int c0 = 0; c0 < D; c0 += 32) {
+          uint32_t r[32];
+          tc::tmem_ld32(lane_base + acc_col(j) + c0, r);
+          tc::tmem_ld_wait();
 #pragma unroll
-            for (int u = 0; u < 32; u += 4) {
-              float o[4];
+          for (int u = 0; u < 32; u += 4) {
+            float o[4];
+            if (EPI == EPI_NODE) {
+              const float4 as4 = *reinterpret_cast<const float4 *>(s.avec + c0 + u);
+              const float4 ad4 = *reinterpret_cast<const float4 *>(s.avec + D + c0 + u);
+              const float asv[4] = {as4.x, as4.y, as4.z, as4.w};
+              const float adv[4] = {ad4.x, ad4.y, ad4.z, ad4.w};
 #pragma unroll
               for (int t = 0; t < 4; ++t) {
-                const float z = __uint_as_float(r[u + t]) * un;
-                if (EPI == EPI_NODE) {
-                  o[t] = lrelu(z, a.slope);
-                  pp = fmaf(o[t], s.avec[c0 + u + t], pp);
-                  qq = fmaf(o[t], s.avec[D + c0 + u + t], qq);
-                } else {
-                  o[t] = 1.f / (1.f + expf(-(aux_prev * z)));          // e' (R2, R3)
-                }
+                o[t] = lrelu(__uint_as_float(r[u + t]) * un, a.slope);
+                pp = fmaf(o[t], asv[t], pp);
+                qq = fmaf(o[t], adv[t], qq);
               }
-              if (live) *reinterpret_cast<float4 *>(orow + c0 + u) = make_float4(o[0], o[1], o[2], o[3]);
+            } else {
+#pragma unroll
+              for (int t = 0; t < 4; ++t)                                      // e' (R2, R3)
+                o[t] = __frcp_rn(1.f + expf(-(aux * (__uint_as_float(r[u + t]) * un))));
             }
-          }
-          if (EPI == EPI_NODE && live) {
-            a.p[grow] = pp;
-            a.q[grow] = qq;
+            if (live) *reinterpret_cast<float4 *>(orow + c0 + u) = make_float4(o[0], o[1], o[2], o[3]);
           }
         }
-        tc::fence_before_sync();
-        tc::mbar_arrive(s.accfree + jp);
+        if (EPI == EPI_NODE && live) {
+          a.p[grow] = pp;
+          a.q[grow] = qq;
+        }
       }
-      e_prev = e_cur;
-      aux_prev = aux_cur;
-      r0_prev = r0;
-      nrows_prev = nrows;
+      tc::fence_before_sync();
     }
   }
   tc::fence_before_sync();
@@ -355,18 +341,25 @@ __global__ void __launch_bounds__(256) edge_small_kernel(
   extern __shared__ float wsm[];            // [D][Ke]
   for (int i = threadIdx.x; i < D * Ke; i += blockDim.x) wsm[i] = W_e[i];
   __syncthreads();
-  constexpr int G = D / 4;                  // lanes per edge
-  const int lanes_total = gridDim.x * blockDim.x;
-  for (long t = blockIdx.x * long(blockDim.x) + threadIdx.x; t < long(E) * G; t += lanes_total) {
-    const long k = t / G;
-    const int c = int(t % G) * 4;
+  constexpr int G = D / 4;                  // lanes per edge (4 channels each)
+  constexpr int EPW = 32 / G;               // edges per warp step
+  const int lane = threadIdx.x & 31;
+  const int sub = lane / G, c = (lane % G) * 4;
+  const long nwarps = long(gridDim.x) * (blockDim.x / 32);
+  for (long k = (blockIdx.x * long(blockDim.x / 32) + threadIdx.x / 32) * EPW + sub; k < E;
+       k += nwarps * EPW) {
     const float al = __ldg(p + in_src[k]) + __ldg(q + in_dst[k]);
+    float e[16];
+#pragma unroll
+    for (int j = 0; j < 16; ++j) e[j] = j < Ke ? __ldg(e_in + k * Ke + j) : 0.f;
     float o[4];
 #pragma unroll
     for (int u = 0; u < 4; ++u) {
       float z = 0.f;
-      for (int j = 0; j < Ke; ++j) z = fmaf(wsm[(c + u) * Ke + j], __ldg(e_in + k * Ke + j), z);
-      o[u] = 1.f / (1.f + expf(-(al * z)));
+#pragma unroll
+      for (int j = 0; j < 16; ++j)
+        if (j < Ke) z = fmaf(wsm[(c + u) * Ke + j], e[j], z);
+      o[u] = __frcp_rn(1.f + expf(-(al * z)));
     }
     *reinterpret_cast<float4 *>(e_out + k * D + c) = make_float4(o[0], o[1], o[2], o[3]);
   }
