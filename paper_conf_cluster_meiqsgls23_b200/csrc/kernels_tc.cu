@@ -47,6 +47,14 @@ constexpr int EPI_NODE = 0, EPI_EDGE = 1, EPI_GATE = 2;
 __device__ __forceinline__ uint32_t a_col(int j) { return uint32_t(j) * 128u; }
 __device__ __forceinline__ uint32_t acc_col(int j) { return 256u + uint32_t(j) * 128u; }
 __device__ __forceinline__ float lrelu(float x, float s) { return x > 0.f ? x : s * x; }
+// Fast exp / reciprocal (MUFU.EX2 / MUFU.RCP, ~2^-22 relative): exact at the
+// closed-form special cases used by the bit-exact tests (exp(0) = 1, 1/2^k).
+__device__ __forceinline__ float fast_exp(float x) { return exp2f(x * 1.4426950408889634f); }
+__device__ __forceinline__ float fast_rcp(float x) {
+  float r;
+  asm("rcp.approx.ftz.f32 %0, %1;" : "=f"(r) : "f"(x));
+  return r;
+}
 
 struct RowGemmArgs {
   const float *A;          // [R][K] input rows (fp32)
@@ -278,10 +286,10 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(RowGemmArgs a) {
         float sum = 0.f;
 #pragma unroll
         for (int c = 0; c < D; ++c) {
-          v[c] = expf(v[c] - m);
+          v[c] = fast_exp(v[c] - m);
           sum += v[c];
         }
-        const float inv = __frcp_rn(sum);
+        const float inv = fast_rcp(sum);
         if (live) {
 #pragma unroll
           for (int c = 0; c < D; c += 4)
@@ -312,7 +320,7 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(RowGemmArgs a) {
             } else {
 #pragma unroll
               for (int t = 0; t < 4; ++t)                                      // e' (R2, R3)
-                o[t] = __frcp_rn(1.f + expf(-(aux * (__uint_as_float(r[u + t]) * un))));
+                o[t] = fast_rcp(1.f + fast_exp(-(aux * (__uint_as_float(r[u + t]) * un))));
             }
             if (live) *reinterpret_cast<float4 *>(orow + c0 + u) = make_float4(o[0], o[1], o[2], o[3]);
           }
@@ -338,8 +346,8 @@ __global__ void __launch_bounds__(256) edge_small_kernel(
     const float *__restrict__ e_in, int Ke, const float *__restrict__ W_e,
     const float *__restrict__ p, const float *__restrict__ q, const int32_t *__restrict__ in_src,
     const int32_t *__restrict__ in_dst, int E, float *__restrict__ e_out) {
-  extern __shared__ float wsm[];            // [D][Ke]
-  for (int i = threadIdx.x; i < D * Ke; i += blockDim.x) wsm[i] = W_e[i];
+  extern __shared__ float wsm[];            // [Ke][D] = W_eᵀ (conflict-free float4 reads)
+  for (int i = threadIdx.x; i < D * Ke; i += blockDim.x) wsm[(i % Ke) * D + i / Ke] = W_e[i];
   __syncthreads();
   constexpr int G = D / 4;                  // lanes per edge (4 channels each)
   constexpr int EPW = 32 / G;               // edges per warp step
@@ -352,15 +360,19 @@ __global__ void __launch_bounds__(256) edge_small_kernel(
     float e[16];
 #pragma unroll
     for (int j = 0; j < 16; ++j) e[j] = j < Ke ? __ldg(e_in + k * Ke + j) : 0.f;
+    float z[4] = {0.f, 0.f, 0.f, 0.f};
+#pragma unroll
+    for (int j = 0; j < 16; ++j)
+      if (j < Ke) {
+        const float4 w = *reinterpret_cast<const float4 *>(wsm + j * D + c);
+        z[0] = fmaf(w.x, e[j], z[0]);
+        z[1] = fmaf(w.y, e[j], z[1]);
+        z[2] = fmaf(w.z, e[j], z[2]);
+        z[3] = fmaf(w.w, e[j], z[3]);
+      }
     float o[4];
 #pragma unroll
-    for (int u = 0; u < 4; ++u) {
-      float z = 0.f;
-#pragma unroll
-      for (int j = 0; j < 16; ++j)
-        if (j < Ke) z = fmaf(wsm[(c + u) * Ke + j], e[j], z);
-      o[u] = __frcp_rn(1.f + expf(-(al * z)));
-    }
+    for (int u = 0; u < 4; ++u) o[u] = fast_rcp(1.f + fast_exp(-(al * z[u])));
     *reinterpret_cast<float4 *>(e_out + k * D + c) = make_float4(o[0], o[1], o[2], o[3]);
   }
 }

@@ -1,0 +1,13 @@
+import json, sys
+for f in sys.argv[1:]:
+    for ln in open(f):
+        if ln.startswith('{'):
+            d = json.loads(ln)
+            print(f, 'value', round(d['value']), 'ms', round(d['ms_per_step'], 4),
+                  'e2e', round(d['e2e']['value']) if d.get('e2e') else None,
+                  'train', d['train'] and round(d['train']['value']))
+            print('  kernels(ms/step)', {k: round(v, 4) for k, v in d['kernel_ms_per_step'].items()})
+            print('  roofline', {k: (round(v, 3) if isinstance(v, float) else v) for k, v in d['roofline'].items()})
+            print('  agg GB/s', d['aggregation']['achieved'], 'clocks', d['clocks'])
+        elif ln.strip():
+            print('  ', ln.strip()[:200])
