@@ -78,13 +78,14 @@ struct Smem {
   int *fexp;
   float *red;
   float *avec;             // [2*D] a_s, a_d (NODE)
+  float *xbuf;             // per worker warp: 16 x 36 floats (coalescing transpose)
 };
 
 __host__ __device__ inline int kpad_of(int K) { return (K + 63) / 64 * 64; }
 __host__ __device__ inline size_t smem_bytes(int D, int K) {
   const size_t img = size_t(kpad_of(K)) * D * 2;
   const size_t slot = size_t(TM) * (K + 4) * 4;
-  return 1024 + 2 * img + 2 * slot + 12 * 8 + 64 + 64 + 2 * D * 4 + 256;
+  return 1024 + 2 * img + 2 * slot + 2048 + 8 * 16 * 36 * 4;
 }
 
 __device__ __forceinline__ Smem carve(uint8_t *raw, int D, int K) {
@@ -106,6 +107,7 @@ __device__ __forceinline__ Smem carve(uint8_t *raw, int D, int K) {
   s.fexp = reinterpret_cast<int *>(bars + 12) + 4;
   s.red = reinterpret_cast<float *>(bars + 12) + 16;
   s.avec = reinterpret_cast<float *>(bars + 12) + 32;
+  s.xbuf = reinterpret_cast<float *>(base + 2 * img + 2 * slot + 2048);
   return s;
 }
 
@@ -124,6 +126,33 @@ __device__ __forceinline__ void split2(float v0, float v1, uint32_t &hi, uint32_
   const __half2 l = __floats2half2_rn(v0 - f.x, v1 - f.y);
   hi = *reinterpret_cast<const uint32_t *>(&h);
   lo = *reinterpret_cast<const uint32_t *>(&l);
+}
+
+// Coalesced store of a 32-column chunk of the warp's 32 rows (thread = row):
+// rows are transposed through a 16 x 36 per-warp buffer so that each warp store
+// instruction writes 4 full 128-byte lines instead of 32 partial ones.
+template <int D>
+__device__ __forceinline__ void warp_store_chunk(float *buf, float *__restrict__ out, long wrow0,
+                                                 int wrows, int c0, const float (&v)[32], int lane) {
+#pragma unroll
+  for (int h = 0; h < 2; ++h) {
+    if ((lane >> 4) == h) {
+      float *b = buf + (lane & 15) * 36;
+#pragma unroll
+      for (int u = 0; u < 32; u += 4)
+        *reinterpret_cast<float4 *>(b + u) = make_float4(v[u], v[u + 1], v[u + 2], v[u + 3]);
+    }
+    __syncwarp();
+#pragma unroll
+    for (int it = 0; it < 4; ++it) {
+      const int idx = it * 32 + lane, r = idx >> 3, c4 = (idx & 7) * 4;
+      const int rr = h * 16 + r;
+      if (rr < wrows)
+        *reinterpret_cast<float4 *>(out + (wrow0 + rr) * D + c0 + c4) =
+            *reinterpret_cast<const float4 *>(buf + r * 36 + c4);
+    }
+    __syncwarp();
+  }
 }
 
 template <int D, int EPI>
@@ -269,7 +298,9 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(RowGemmArgs a) {
       tc::fence_after_sync();
       const float un = ldexpf(1.f, -(er + fexp));
       const long grow = r0 + row;
-      float *orow = a.out + grow * D;
+      float *wbuf = s.xbuf + (warp - 2) * (16 * 36);
+      const long wrow0 = r0 + qd * 32;
+      const int wrows = max(0, min(32, nrows - qd * 32));
       if (EPI == EPI_GATE) {
         float v[D];
 #pragma unroll
@@ -290,11 +321,12 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(RowGemmArgs a) {
           sum += v[c];
         }
         const float inv = fast_rcp(sum);
-        if (live) {
 #pragma unroll
-          for (int c = 0; c < D; c += 4)
-            *reinterpret_cast<float4 *>(orow + c) =
-                make_float4(v[c] * inv, v[c + 1] * inv, v[c + 2] * inv, v[c + 3] * inv);
+        for (int c0 = 0; c0 < D; c0 += 32) {
+          float o[32];
+#pragma unroll
+          for (int u = 0; u < 32; ++u) o[u] = v[c0 + u] * inv;
+          warp_store_chunk<D>(wbuf, a.out, wrow0, wrows, c0, o, lane);
         }
       } else {
         float pp = 0.f, qq = 0.f;
@@ -303,9 +335,9 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(RowGemmArgs a) {
           uint32_t r[32];
           tc::tmem_ld32(lane_base + acc_col(j) + c0, r);
           tc::tmem_ld_wait();
+          float o[32];
 #pragma unroll
           for (int u = 0; u < 32; u += 4) {
-            float o[4];
             if (EPI == EPI_NODE) {
               const float4 as4 = *reinterpret_cast<const float4 *>(s.avec + c0 + u);
               const float4 ad4 = *reinterpret_cast<const float4 *>(s.avec + D + c0 + u);
@@ -313,17 +345,17 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(RowGemmArgs a) {
               const float adv[4] = {ad4.x, ad4.y, ad4.z, ad4.w};
 #pragma unroll
               for (int t = 0; t < 4; ++t) {
-                o[t] = lrelu(__uint_as_float(r[u + t]) * un, a.slope);
-                pp = fmaf(o[t], asv[t], pp);
-                qq = fmaf(o[t], adv[t], qq);
+                o[u + t] = lrelu(__uint_as_float(r[u + t]) * un, a.slope);
+                pp = fmaf(o[u + t], asv[t], pp);
+                qq = fmaf(o[u + t], adv[t], qq);
               }
             } else {
 #pragma unroll
               for (int t = 0; t < 4; ++t)                                      // e' (R2, R3)
-                o[t] = fast_rcp(1.f + fast_exp(-(aux * (__uint_as_float(r[u + t]) * un))));
+                o[u + t] = fast_rcp(1.f + fast_exp(-(aux * (__uint_as_float(r[u + t]) * un))));
             }
-            if (live) *reinterpret_cast<float4 *>(orow + c0 + u) = make_float4(o[0], o[1], o[2], o[3]);
           }
+          warp_store_chunk<D>(wbuf, a.out, wrow0, wrows, c0, o, lane);
         }
         if (EPI == EPI_NODE && live) {
           a.p[grow] = pp;
