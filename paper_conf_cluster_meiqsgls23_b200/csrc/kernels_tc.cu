@@ -82,9 +82,11 @@ struct Smem {
 };
 
 __host__ __device__ inline int kpad_of(int K) { return (K + 63) / 64 * 64; }
+// input slot: ceil(K/32) TMA boxes of 128 rows x 32 fp32 (128 B, SW128-swizzled)
+__host__ __device__ inline int nbox_of(int K) { return (K + 31) / 32; }
 __host__ __device__ inline size_t smem_bytes(int D, int K) {
   const size_t img = size_t(kpad_of(K)) * D * 2;
-  const size_t slot = size_t(TM) * (K + 4) * 4;
+  const size_t slot = size_t(nbox_of(K)) * 16384;
   return 1024 + 2 * img + 2 * slot + 2048 + 8 * 16 * 36 * 4;
 }
 
@@ -93,7 +95,7 @@ __device__ __forceinline__ Smem carve(uint8_t *raw, int D, int K) {
   const uint32_t a = tc::smem_u32(raw);
   uint8_t *base = raw + ((1024 - (a & 1023)) & 1023);
   const size_t img = size_t(kpad_of(K)) * D * 2;
-  const size_t slot = size_t(TM) * (K + 4) * 4;
+  const size_t slot = size_t(nbox_of(K)) * 16384;
   s.w0 = base;
   s.w1 = base + img;
   s.slot0 = reinterpret_cast<float *>(base + 2 * img);
@@ -155,10 +157,17 @@ __device__ __forceinline__ void warp_store_chunk(float *buf, float *__restrict__
   }
 }
 
+// float4 of row r, columns [k, k+4) (k % 4 == 0) inside a slot of SW128 TMA boxes.
+__device__ __forceinline__ float4 slot_ld4(const float *slot, int r, int k) {
+  const int b = k >> 5, c = (k & 31) >> 2;
+  return *reinterpret_cast<const float4 *>(slot + b * 4096 + r * 32 + ((c ^ (r & 7)) << 2));
+}
+
 template <int D, int EPI>
-__global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(RowGemmArgs a) {
+__global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__ CUtensorMap tmap,
+                                                         RowGemmArgs a) {
   extern __shared__ uint8_t smem_raw[];
-  const int K = a.K, Kpad = kpad_of(K), S = K + 4;
+  const int K = a.K, Kpad = kpad_of(K), NB = nbox_of(K);
   Smem s = carve(smem_raw, D, K);
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
 
@@ -213,17 +222,18 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(RowGemmArgs a) {
   const int my = blockIdx.x < tiles ? (tiles - 1 - int(blockIdx.x)) / int(gridDim.x) + 1 : 0;
 
   if (warp == 0) {
-    // ---------------- producer: tile i -> slot i%2 ----------------
-    for (int i = 0; i < my; ++i) {
-      const int j = i & 1;
-      const long r0 = long(blockIdx.x + i * gridDim.x) * TM;
-      const int nrows = min(TM, int(a.R - r0));
-      if (i >= 2) tc::mbar_wait(s.empty + j, ((i >> 1) - 1) & 1);
-      if (lane == 0) tc::mbar_arrive_expect_tx(s.full + j, uint32_t(nrows) * K * 4);
-      __syncwarp();
-      for (int r = lane; r < nrows; r += 32)
-        tc::bulk_g2s(s.slot(j) + r * S, a.A + (r0 + r) * K, uint32_t(K) * 4, s.full + j);
+    // ---------------- producer: tile i -> slot i%2 (TMA 2D, OOB rows zero-filled) -------
+    if (lane == 0) {
+      tc::prefetch_tmap(&tmap);
+      for (int i = 0; i < my; ++i) {
+        const int j = i & 1;
+        const int r0 = int(blockIdx.x + i * gridDim.x) * TM;
+        if (i >= 2) tc::mbar_wait(s.empty + j, ((i >> 1) - 1) & 1);
+        tc::mbar_arrive_expect_tx(s.full + j, uint32_t(NB) * 16384u);
+        for (int b = 0; b < NB; ++b) tc::tma_load_2d(s.slot(j) + b * 4096, &tmap, 32 * b, r0, s.full + j);
+      }
     }
+    __syncwarp();
   } else if (warp == 1) {
     // ---------------- MMA issuer: tiles in order, A[i%2] -> ACC[i%2] ----------------
     const uint32_t idsc = tc::idesc(128, uint32_t(D), tc::FMT_F16);
@@ -266,12 +276,12 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(RowGemmArgs a) {
         aux = __ldg(a.pin + a.src[r0 + row]) + __ldg(a.qin + a.dst[r0 + row]);   // α (R1)
       // -- convert the row into TMEM A[j] (its previous MMA finished: we consumed ACC[j])
       tc::mbar_wait(s.full + j, par);
-      const float *rp = s.slot(j) + row * S;
+      const float *sl = s.slot(j);
       float mx = 0.f;
       if (live)
 #pragma unroll 8
         for (int k = 0; k < K; k += 4) {
-          const float4 v = *reinterpret_cast<const float4 *>(rp + k);
+          const float4 v = slot_ld4(sl, row, k);
           mx = fmaxf(mx, fmaxf(fmaxf(fabsf(v.x), fabsf(v.y)), fmaxf(fabsf(v.z), fabsf(v.w))));
         }
       const int er = scale_exp(mx);
@@ -282,7 +292,7 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(RowGemmArgs a) {
         for (int u = 0; u < 32; u += 2) {
           const int k = 2 * (c0 + u);
           float4 v = make_float4(0.f, 0.f, 0.f, 0.f);
-          if (live && k < K) v = *reinterpret_cast<const float4 *>(rp + k);
+          if (live && k < K) v = slot_ld4(sl, row, k);
           split2(v.x * xs, v.y * xs, x0[u], x1[u]);
           split2(v.z * xs, v.w * xs, x0[u + 1], x1[u + 1]);
         }
@@ -409,6 +419,32 @@ __global__ void __launch_bounds__(256) edge_small_kernel(
   }
 }
 
+typedef CUresult (*PFN_encodeTiled)(CUtensorMap *, CUtensorMapDataType, cuuint32_t, void *,
+                                    const cuuint64_t *, const cuuint64_t *, const cuuint32_t *,
+                                    const cuuint32_t *, CUtensorMapInterleave, CUtensorMapSwizzle,
+                                    CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+
+// Tensor map of a row-major fp32 matrix [R][K]: boxes of 128 rows x 32 columns,
+// 128-byte swizzle, out-of-bounds elements read as zero.
+bool encode_rows_map(CUtensorMap *m, const float *A, int R, int K) {
+  static PFN_encodeTiled fn = nullptr;
+  if (!fn) {
+    void *p = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) != cudaSuccess ||
+        q != cudaDriverEntryPointSuccess || !p)
+      return false;
+    fn = reinterpret_cast<PFN_encodeTiled>(p);
+  }
+  const cuuint64_t dims[2] = {cuuint64_t(K), cuuint64_t(R)};
+  const cuuint64_t strides[1] = {cuuint64_t(K) * 4};
+  const cuuint32_t box[2] = {32, 128};
+  const cuuint32_t estr[2] = {1, 1};
+  return fn(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, const_cast<float *>(A), dims, strides, box, estr,
+            CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+            CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
 template <class Kern> void set_smem(Kern k, size_t bytes) {
   cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, int(bytes));
 }
@@ -435,8 +471,10 @@ static int launch_rowgemm(const occu_ctx *ctx, const RowGemmArgs &ra, const char
   set_smem(rowgemm_kernel<D, EPI>, smem);
   const int tiles = (ra.R + TM - 1) / TM;
   const int grid = std::min(tiles, ctx->num_sms);
+  CUtensorMap tmap;
+  if (!encode_rows_map(&tmap, ra.A, ra.R, ra.K)) return -int(cudaErrorInvalidValue);
   OCCU_PROF_BEGIN(ctx, name, st);
-  rowgemm_kernel<D, EPI><<<grid, NTH, smem, st>>>(ra);
+  rowgemm_kernel<D, EPI><<<grid, NTH, smem, st>>>(tmap, ra);
   OCCU_PROF_END(ctx);
   TC_CHECK();
   return 1;
