@@ -40,9 +40,26 @@ namespace occu {
 namespace {
 
 constexpr int TM = 128;
-constexpr int NTH = 320;
+constexpr int NTH = 576;          // warp 0 producer, warp 1 MMA, warps 2-17 workers
 constexpr uint32_t TMEM_COLS = 512;
 constexpr int EPI_NODE = 0, EPI_EDGE = 1, EPI_GATE = 2;
+
+#ifdef OCCU_TC_TRACE
+// Debug timeline: CTA 0 records clock64 stamps (role, tile, event) into g_trace.
+__device__ long long g_trace[4096][4];
+__device__ int g_trace_n;
+template <int EPI> __device__ __forceinline__ void trace(int role, int tile, int ev) {
+  if (EPI == OCCU_TC_TRACE && blockIdx.x == 0 && (threadIdx.x & 31) == 0) {
+    const int k = atomicAdd(&g_trace_n, 1);
+    if (k < 4096) {
+      g_trace[k][0] = clock64(); g_trace[k][1] = role; g_trace[k][2] = tile; g_trace[k][3] = ev;
+    }
+  }
+}
+#define TRACE(role, tile, ev) trace<EPI>(role, tile, ev)
+#else
+#define TRACE(role, tile, ev)
+#endif
 
 __device__ __forceinline__ uint32_t a_col(int j) { return uint32_t(j) * 128u; }
 __device__ __forceinline__ uint32_t acc_col(int j) { return 256u + uint32_t(j) * 128u; }
@@ -78,7 +95,8 @@ struct Smem {
   int *fexp;
   float *red;
   float *avec;             // [2*D] a_s, a_d (NODE)
-  float *xbuf;             // per worker warp: 16 x 36 floats (coalescing transpose)
+  float *xbuf;             // per worker warp: 8 x 36 floats (coalescing transpose)
+  float *xch;              // [2 groups][2 values][2 halves][128 rows] row-partial exchange
 };
 
 __host__ __device__ inline int kpad_of(int K) { return (K + 63) / 64 * 64; }
@@ -87,7 +105,7 @@ __host__ __device__ inline int nbox_of(int K) { return (K + 31) / 32; }
 __host__ __device__ inline size_t smem_bytes(int D, int K) {
   const size_t img = size_t(kpad_of(K)) * D * 2;
   const size_t slot = size_t(nbox_of(K)) * 16384;
-  return 1024 + 2 * img + 2 * slot + 2048 + 8 * 16 * 36 * 4;
+  return 1024 + 2 * img + 2 * slot + 2048 + 16 * 8 * 36 * 4 + 2 * 2 * 2 * 128 * 4;
 }
 
 __device__ __forceinline__ Smem carve(uint8_t *raw, int D, int K) {
@@ -110,6 +128,7 @@ __device__ __forceinline__ Smem carve(uint8_t *raw, int D, int K) {
   s.red = reinterpret_cast<float *>(bars + 12) + 16;
   s.avec = reinterpret_cast<float *>(bars + 12) + 32;
   s.xbuf = reinterpret_cast<float *>(base + 2 * img + 2 * slot + 2048);
+  s.xch = s.xbuf + 16 * 8 * 36;
   return s;
 }
 
@@ -131,30 +150,34 @@ __device__ __forceinline__ void split2(float v0, float v1, uint32_t &hi, uint32_
 }
 
 // Coalesced store of a 32-column chunk of the warp's 32 rows (thread = row):
-// rows are transposed through a 16 x 36 per-warp buffer so that each warp store
+// rows are transposed through an 8 x 36 per-warp buffer so that each warp store
 // instruction writes 4 full 128-byte lines instead of 32 partial ones.
 template <int D>
 __device__ __forceinline__ void warp_store_chunk(float *buf, float *__restrict__ out, long wrow0,
                                                  int wrows, int c0, const float (&v)[32], int lane) {
 #pragma unroll
-  for (int h = 0; h < 2; ++h) {
-    if ((lane >> 4) == h) {
-      float *b = buf + (lane & 15) * 36;
+  for (int h = 0; h < 4; ++h) {
+    if ((lane >> 3) == h) {
+      float *b = buf + (lane & 7) * 36;
 #pragma unroll
       for (int u = 0; u < 32; u += 4)
         *reinterpret_cast<float4 *>(b + u) = make_float4(v[u], v[u + 1], v[u + 2], v[u + 3]);
     }
     __syncwarp();
 #pragma unroll
-    for (int it = 0; it < 4; ++it) {
+    for (int it = 0; it < 2; ++it) {
       const int idx = it * 32 + lane, r = idx >> 3, c4 = (idx & 7) * 4;
-      const int rr = h * 16 + r;
+      const int rr = h * 8 + r;
       if (rr < wrows)
         *reinterpret_cast<float4 *>(out + (wrow0 + rr) * D + c0 + c4) =
             *reinterpret_cast<const float4 *>(buf + r * 36 + c4);
     }
     __syncwarp();
   }
+}
+
+__device__ __forceinline__ void group_bar(int g) {
+  asm volatile("bar.sync %0, 256;" ::"r"(1 + g) : "memory");
 }
 
 // float4 of row r, columns [k, k+4) (k % 4 == 0) inside a slot of SW128 TMA boxes.
@@ -204,8 +227,8 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
   if (threadIdx.x == 0) {
     for (int j = 0; j < 2; ++j) {
       tc::mbar_init(s.full + j, 1);
-      tc::mbar_init(s.empty + j, 128);
-      tc::mbar_init(s.afull + j, 128);
+      tc::mbar_init(s.empty + j, 256);
+      tc::mbar_init(s.afull + j, 256);
       tc::mbar_init(s.accfull + j, 1);
     }
     tc::fence_mbar_init();
@@ -228,7 +251,9 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
       for (int i = 0; i < my; ++i) {
         const int j = i & 1;
         const int r0 = int(blockIdx.x + i * gridDim.x) * TM;
+        TRACE(0, i, 0);
         if (i >= 2) tc::mbar_wait(s.empty + j, ((i >> 1) - 1) & 1);
+        TRACE(0, i, 1);
         tc::mbar_arrive_expect_tx(s.full + j, uint32_t(NB) * 16384u);
         for (int b = 0; b < NB; ++b) tc::tma_load_2d(s.slot(j) + b * 4096, &tmap, 32 * b, r0, s.full + j);
       }
@@ -241,7 +266,9 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
     const int nk = (K + 15) / 16;
     for (int i = 0; i < my; ++i) {
       const int j = i & 1;
+      TRACE(1, i, 0);
       tc::mbar_wait(s.afull + j, (i >> 1) & 1);
+      TRACE(1, i, 1);
       tc::fence_after_sync();
       if (lane == 0) {
         const uint32_t d = tmem + acc_col(j);
@@ -259,98 +286,135 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
       __syncwarp();
     }
   } else {
-    // ---------------- workers: two ping-pong warpgroups (warps 2-5, 6-9) -------------
-    // group g handles local tiles i = g, g+2, ... : convert -> MMA -> epilogue, thread = row.
-    const int g = (warp - 2) >> 2;
-    const int qd = warp & 3;                       // TMEM lane quarter of this warp
+    // ---------------- workers: two ping-pong groups of 8 warps (warps 2-9, 10-17) -------
+    // group g handles local tiles i = g, g+2, ...; a row is shared by two warps of the
+    // same TMEM lane quarter (warp % 4): half hf owns K-columns / output columns
+    // [hf*X/2, (hf+1)*X/2).  Row-wide quantities (scale, softmax max/sum, p, q) are
+    // combined through smem with a 256-thread named barrier per group.
+    const int wi = warp - 2;
+    const int g = wi >> 3;
+    const int hf = (wi >> 2) & 1;
+    const int qd = warp & 3;
     const int row = qd * 32 + lane;
     const uint32_t lane_base = tmem + (uint32_t(qd * 32) << 16);
+    float *xg = s.xch + g * (2 * 2 * 128);           // [value][half][row]
+    float *wbuf = s.xbuf + wi * (8 * 36);
+    const int KH = Kpad / 2;                          // K-elements per half (Kpad = 64 or 128)
     for (int i = g; i < my; i += 2) {
-      const int j = i & 1;                         // == g
+      const int j = i & 1;
       const uint32_t par = (i >> 1) & 1;
       const long r0 = long(blockIdx.x + i * gridDim.x) * TM;
       const int nrows = min(TM, int(a.R - r0));
       const bool live = row < nrows;
-      float aux = 0.f;
-      if (EPI == EPI_EDGE && live)
-        aux = __ldg(a.pin + a.src[r0 + row]) + __ldg(a.qin + a.dst[r0 + row]);   // α (R1)
-      // -- convert the row into TMEM A[j] (its previous MMA finished: we consumed ACC[j])
+      int sidx = 0, didx = 0;
+      if (EPI == EPI_EDGE && live && hf == 0) {
+        sidx = __ldg(a.src + r0 + row);
+        didx = __ldg(a.dst + r0 + row);
+      }
+      // -- convert this thread's half row into TMEM A[j]
+      TRACE(2 + warp, i, 0);
       tc::mbar_wait(s.full + j, par);
+      TRACE(2 + warp, i, 1);
       const float *sl = s.slot(j);
+      const int kb = hf * KH, ke = min(K, kb + KH);
       float mx = 0.f;
       if (live)
-#pragma unroll 8
-        for (int k = 0; k < K; k += 4) {
+#pragma unroll 4
+        for (int k = kb; k < ke; k += 4) {
           const float4 v = slot_ld4(sl, row, k);
           mx = fmaxf(mx, fmaxf(fmaxf(fabsf(v.x), fabsf(v.y)), fmaxf(fabsf(v.z), fabsf(v.w))));
         }
+      xg[hf * 128 + row] = mx;
+      group_bar(g);
+      mx = fmaxf(mx, xg[(hf ^ 1) * 128 + row]);
       const int er = scale_exp(mx);
       const float xs = ldexpf(1.f, er);
-      for (int c0 = 0; c0 < Kpad / 2; c0 += 32) {
+      for (int c0 = 0; c0 < KH / 2; c0 += 32) {       // TMEM columns of this half
         uint32_t x0[32], x1[32];
 #pragma unroll
         for (int u = 0; u < 32; u += 2) {
-          const int k = 2 * (c0 + u);
+          const int k = kb + 2 * (c0 + u);
           float4 v = make_float4(0.f, 0.f, 0.f, 0.f);
           if (live && k < K) v = slot_ld4(sl, row, k);
           split2(v.x * xs, v.y * xs, x0[u], x1[u]);
           split2(v.z * xs, v.w * xs, x0[u + 1], x1[u + 1]);
         }
-        tc::tmem_st32(lane_base + a_col(j) + c0, x0);
-        tc::tmem_st32(lane_base + a_col(j) + Kpad / 2 + c0, x1);
+        const uint32_t col = a_col(j) + uint32_t(kb / 2 + c0);
+        tc::tmem_st32(lane_base + col, x0);
+        tc::tmem_st32(lane_base + col + Kpad / 2, x1);
       }
       tc::tmem_st_wait();
       tc::fence_before_sync();
       tc::mbar_arrive(s.empty + j);
       tc::mbar_arrive(s.afull + j);
-      // -- epilogue
+      float aux = 0.f;
+      if (EPI == EPI_EDGE) {                          // α = p[s] + q[t] (R1), exchanged
+        if (hf == 0) {
+          aux = live ? __ldg(a.pin + sidx) + __ldg(a.qin + didx) : 0.f;
+          xg[row] = aux;
+        }
+      }
+      // -- epilogue over output columns [hf*D/2, (hf+1)*D/2)
+      TRACE(2 + warp, i, 2);
       tc::mbar_wait(s.accfull + j, par);
+      TRACE(2 + warp, i, 3);
       tc::fence_after_sync();
+      if (EPI == EPI_EDGE) {
+        group_bar(g);
+        aux = xg[row];
+      }
       const float un = ldexpf(1.f, -(er + fexp));
       const long grow = r0 + row;
-      float *wbuf = s.xbuf + (warp - 2) * (16 * 36);
       const long wrow0 = r0 + qd * 32;
       const int wrows = max(0, min(32, nrows - qd * 32));
+      constexpr int DH = D / 2;
+      const int cb = hf * DH;
       if (EPI == EPI_GATE) {
-        float v[D];
+        float v[DH];
 #pragma unroll
-        for (int c0 = 0; c0 < D; c0 += 32) {
+        for (int c0 = 0; c0 < DH; c0 += 32) {
           uint32_t r[32];
-          tc::tmem_ld32(lane_base + acc_col(j) + c0, r);
+          tc::tmem_ld32(lane_base + acc_col(j) + cb + c0, r);
           tc::tmem_ld_wait();
 #pragma unroll
           for (int u = 0; u < 32; ++u) v[c0 + u] = __uint_as_float(r[u]) * un;
         }
         float m = -INFINITY;
 #pragma unroll
-        for (int c = 0; c < D; ++c) m = fmaxf(m, v[c]);
+        for (int c = 0; c < DH; ++c) m = fmaxf(m, v[c]);
+        xg[hf * 128 + row] = m;
+        group_bar(g);
+        m = fmaxf(m, xg[(hf ^ 1) * 128 + row]);
         float sum = 0.f;
 #pragma unroll
-        for (int c = 0; c < D; ++c) {
+        for (int c = 0; c < DH; ++c) {
           v[c] = fast_exp(v[c] - m);
           sum += v[c];
         }
+        xg[256 + hf * 128 + row] = sum;
+        group_bar(g);
+        sum = hf == 0 ? sum + xg[256 + 128 + row] : xg[256 + row] + sum;   // fixed order
         const float inv = fast_rcp(sum);
 #pragma unroll
-        for (int c0 = 0; c0 < D; c0 += 32) {
+        for (int c0 = 0; c0 < DH; c0 += 32) {
           float o[32];
 #pragma unroll
           for (int u = 0; u < 32; ++u) o[u] = v[c0 + u] * inv;
-          warp_store_chunk<D>(wbuf, a.out, wrow0, wrows, c0, o, lane);
+          warp_store_chunk<D>(wbuf, a.out, wrow0, wrows, cb + c0, o, lane);
         }
       } else {
         float pp = 0.f, qq = 0.f;
 #pragma unroll
-        for (int c0 = 0; c0 < D; c0 += 32) {
+        for (int c0 = 0; c0 < DH; c0 += 32) {
           uint32_t r[32];
-          tc::tmem_ld32(lane_base + acc_col(j) + c0, r);
+          tc::tmem_ld32(lane_base + acc_col(j) + cb + c0, r);
           tc::tmem_ld_wait();
           float o[32];
 #pragma unroll
           for (int u = 0; u < 32; u += 4) {
             if (EPI == EPI_NODE) {
-              const float4 as4 = *reinterpret_cast<const float4 *>(s.avec + c0 + u);
-              const float4 ad4 = *reinterpret_cast<const float4 *>(s.avec + D + c0 + u);
+              const float4 as4 = *reinterpret_cast<const float4 *>(s.avec + cb + c0 + u);
+              const float4 ad4 = *reinterpret_cast<const float4 *>(s.avec + D + cb + c0 + u);
               const float asv[4] = {as4.x, as4.y, as4.z, as4.w};
               const float adv[4] = {ad4.x, ad4.y, ad4.z, ad4.w};
 #pragma unroll
@@ -365,14 +429,21 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
                 o[u + t] = fast_rcp(1.f + fast_exp(-(aux * (__uint_as_float(r[u + t]) * un))));
             }
           }
-          warp_store_chunk<D>(wbuf, a.out, wrow0, wrows, c0, o, lane);
+          warp_store_chunk<D>(wbuf, a.out, wrow0, wrows, cb + c0, o, lane);
         }
-        if (EPI == EPI_NODE && live) {
-          a.p[grow] = pp;
-          a.q[grow] = qq;
+        if (EPI == EPI_NODE) {
+          xg[hf * 128 + row] = pp;
+          xg[256 + hf * 128 + row] = qq;
+          group_bar(g);
+          if (hf == 0 && live) {
+            a.p[grow] = pp + xg[128 + row];
+            a.q[grow] = qq + xg[256 + 128 + row];
+          }
         }
       }
+      TRACE(2 + warp, i, 4);
       tc::fence_before_sync();
+      group_bar(g);        // the exchange buffer is reused by the next tile
     }
   }
   tc::fence_before_sync();
@@ -534,3 +605,17 @@ int launch_forward_layer_tc(const occu_ctx *ctx, const DevCsr &csr, const FwdLay
 }
 
 }  // namespace occu
+
+#ifdef OCCU_TC_TRACE
+extern "C" int occu_debug_trace(long long *host, int max_events) {
+  int n = 0;
+  cudaDeviceSynchronize();
+  cudaMemcpyFromSymbol(&n, occu::g_trace_n, sizeof(int));
+  n = n < max_events ? n : max_events;
+  n = n < 4096 ? n : 4096;
+  cudaMemcpyFromSymbol(host, occu::g_trace, size_t(n) * 4 * sizeof(long long));
+  const int zero = 0;
+  cudaMemcpyToSymbol(occu::g_trace_n, &zero, sizeof(int));
+  return n;
+}
+#endif
