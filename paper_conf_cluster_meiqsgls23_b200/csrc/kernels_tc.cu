@@ -32,6 +32,7 @@
 #include <stdint.h>
 
 #include <algorithm>
+#include <cstdlib>
 
 #include "occu_internal.h"
 #include "tc_common.cuh"
@@ -40,26 +41,11 @@ namespace occu {
 namespace {
 
 constexpr int TM = 128;
-constexpr int NTH = 576;          // warp 0 producer, warp 1 MMA, warps 2-17 workers
+constexpr int NTH = 704;          // warp 0 producer, 1 MMA, 2-5 converters, 6-21 epilogue
 constexpr uint32_t TMEM_COLS = 512;
 constexpr int EPI_NODE = 0, EPI_EDGE = 1, EPI_GATE = 2;
 
-#ifdef OCCU_TC_TRACE
-// Debug timeline: CTA 0 records clock64 stamps (role, tile, event) into g_trace.
-__device__ long long g_trace[4096][4];
-__device__ int g_trace_n;
-template <int EPI> __device__ __forceinline__ void trace(int role, int tile, int ev) {
-  if (EPI == OCCU_TC_TRACE && blockIdx.x == 0 && (threadIdx.x & 31) == 0) {
-    const int k = atomicAdd(&g_trace_n, 1);
-    if (k < 4096) {
-      g_trace[k][0] = clock64(); g_trace[k][1] = role; g_trace[k][2] = tile; g_trace[k][3] = ev;
-    }
-  }
-}
-#define TRACE(role, tile, ev) trace<EPI>(role, tile, ev)
-#else
-#define TRACE(role, tile, ev)
-#endif
+
 
 __device__ __forceinline__ uint32_t a_col(int j) { return uint32_t(j) * 128u; }
 __device__ __forceinline__ uint32_t acc_col(int j) { return 256u + uint32_t(j) * 128u; }
@@ -90,11 +76,12 @@ struct Smem {
   float *slot0;
   int slot_floats;
   __device__ __forceinline__ float *slot(int j) const { return slot0 + j * slot_floats; }
-  uint64_t *full, *empty, *afull, *accfull;
+  uint64_t *full, *empty, *afull, *afree, *accfull, *accfree, *eready;
   uint32_t *tmem_slot;
   int *fexp;
   float *red;
   float *avec;             // [2*D] a_s, a_d (NODE)
+  int *erow;               // [4][128] per-row scale exponents, converter -> epilogue
   float *xbuf;             // per worker warp: 8 x 36 floats (coalescing transpose)
   float *xch;              // [2 groups][2 values][2 halves][128 rows] row-partial exchange
 };
@@ -105,7 +92,7 @@ __host__ __device__ inline int nbox_of(int K) { return (K + 31) / 32; }
 __host__ __device__ inline size_t smem_bytes(int D, int K) {
   const size_t img = size_t(kpad_of(K)) * D * 2;
   const size_t slot = size_t(nbox_of(K)) * 16384;
-  return 1024 + 2 * img + 2 * slot + 2048 + 16 * 8 * 36 * 4 + 2 * 2 * 2 * 128 * 4;
+  return 1024 + 2 * img + 2 * slot + 4096 + 16 * 8 * 36 * 4 + 2 * 2 * 2 * 128 * 4;
 }
 
 __device__ __forceinline__ Smem carve(uint8_t *raw, int D, int K) {
@@ -118,16 +105,21 @@ __device__ __forceinline__ Smem carve(uint8_t *raw, int D, int K) {
   s.w1 = base + img;
   s.slot0 = reinterpret_cast<float *>(base + 2 * img);
   s.slot_floats = int(slot / 4);
-  uint64_t *bars = reinterpret_cast<uint64_t *>(base + 2 * img + 2 * slot);
+  uint8_t *misc = base + 2 * img + 2 * slot;
+  uint64_t *bars = reinterpret_cast<uint64_t *>(misc);
   s.full = bars;
   s.empty = bars + 2;
   s.afull = bars + 4;
+  s.afree = bars + 6;
   s.accfull = bars + 8;
-  s.tmem_slot = reinterpret_cast<uint32_t *>(bars + 12);
-  s.fexp = reinterpret_cast<int *>(bars + 12) + 4;
-  s.red = reinterpret_cast<float *>(bars + 12) + 16;
-  s.avec = reinterpret_cast<float *>(bars + 12) + 32;
-  s.xbuf = reinterpret_cast<float *>(base + 2 * img + 2 * slot + 2048);
+  s.accfree = bars + 10;
+  s.eready = bars + 12;                 // 4
+  s.tmem_slot = reinterpret_cast<uint32_t *>(misc + 128);
+  s.fexp = reinterpret_cast<int *>(misc + 132);
+  s.red = reinterpret_cast<float *>(misc + 256);
+  s.avec = reinterpret_cast<float *>(misc + 512);
+  s.erow = reinterpret_cast<int *>(misc + 1536);
+  s.xbuf = reinterpret_cast<float *>(misc + 4096);
   s.xch = s.xbuf + 16 * 8 * 36;
   return s;
 }
@@ -227,10 +219,13 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
   if (threadIdx.x == 0) {
     for (int j = 0; j < 2; ++j) {
       tc::mbar_init(s.full + j, 1);
-      tc::mbar_init(s.empty + j, 256);
-      tc::mbar_init(s.afull + j, 256);
+      tc::mbar_init(s.empty + j, 128);
+      tc::mbar_init(s.afull + j, 128);
+      tc::mbar_init(s.afree + j, 1);
       tc::mbar_init(s.accfull + j, 1);
+      tc::mbar_init(s.accfree + j, 256);
     }
+    for (int j = 0; j < 4; ++j) tc::mbar_init(s.eready + j, 128);
     tc::fence_mbar_init();
   }
   if (warp == 1) tc::tmem_alloc<TMEM_COLS>(s.tmem_slot);
@@ -251,24 +246,21 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
       for (int i = 0; i < my; ++i) {
         const int j = i & 1;
         const int r0 = int(blockIdx.x + i * gridDim.x) * TM;
-        TRACE(0, i, 0);
         if (i >= 2) tc::mbar_wait(s.empty + j, ((i >> 1) - 1) & 1);
-        TRACE(0, i, 1);
         tc::mbar_arrive_expect_tx(s.full + j, uint32_t(NB) * 16384u);
         for (int b = 0; b < NB; ++b) tc::tma_load_2d(s.slot(j) + b * 4096, &tmap, 32 * b, r0, s.full + j);
       }
     }
     __syncwarp();
   } else if (warp == 1) {
-    // ---------------- MMA issuer: tiles in order, A[i%2] -> ACC[i%2] ----------------
+    // ---------------- MMA issuer: A[i%2] -> ACC[i%2] ----------------
     const uint32_t idsc = tc::idesc(128, uint32_t(D), tc::FMT_F16);
     const uint32_t w0a = tc::smem_u32(s.w0), w1a = tc::smem_u32(s.w1);
     const int nk = (K + 15) / 16;
     for (int i = 0; i < my; ++i) {
       const int j = i & 1;
-      TRACE(1, i, 0);
       tc::mbar_wait(s.afull + j, (i >> 1) & 1);
-      TRACE(1, i, 1);
+      if (i >= 2) tc::mbar_wait(s.accfree + j, ((i >> 1) - 1) & 1);
       tc::fence_after_sync();
       if (lane == 0) {
         const uint32_t d = tmem + acc_col(j);
@@ -282,16 +274,56 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
           tc::mma_f16_ts(d, a1, b0, idsc, 1u);
         }
         tc::mma_commit(s.accfull + j);
+        tc::mma_commit(s.afree + j);
       }
       __syncwarp();
     }
+  } else if (warp < 6) {
+    // ---------------- converters (warps 2-5), thread = row: slot -> TMEM A ----------------
+    const int qd = warp & 3;
+    const int row = qd * 32 + lane;
+    const uint32_t lane_base = tmem + (uint32_t(qd * 32) << 16);
+    for (int i = 0; i < my; ++i) {
+      const int j = i & 1;
+      const long r0 = long(blockIdx.x + i * gridDim.x) * TM;
+      const bool live = row < min(TM, int(a.R - r0));
+      tc::mbar_wait(s.full + j, (i >> 1) & 1);
+      if (i >= 2) tc::mbar_wait(s.afree + j, ((i >> 1) - 1) & 1);
+      const float *sl = s.slot(j);
+      float mx = 0.f;
+      if (live)
+#pragma unroll 8
+        for (int k = 0; k < K; k += 4) {
+          const float4 v = slot_ld4(sl, row, k);
+          mx = fmaxf(mx, fmaxf(fmaxf(fabsf(v.x), fabsf(v.y)), fmaxf(fabsf(v.z), fabsf(v.w))));
+        }
+      const int er = scale_exp(mx);
+      const float xs = ldexpf(1.f, er);
+      for (int c0 = 0; c0 < Kpad / 2; c0 += 32) {
+        uint32_t x0[32], x1[32];
+#pragma unroll
+        for (int u = 0; u < 32; u += 2) {
+          const int k = 2 * (c0 + u);
+          float4 v = make_float4(0.f, 0.f, 0.f, 0.f);
+          if (live && k < K) v = slot_ld4(sl, row, k);
+          split2(v.x * xs, v.y * xs, x0[u], x1[u]);
+          split2(v.z * xs, v.w * xs, x0[u + 1], x1[u + 1]);
+        }
+        tc::tmem_st32(lane_base + a_col(j) + c0, x0);
+        tc::tmem_st32(lane_base + a_col(j) + Kpad / 2 + c0, x1);
+      }
+      s.erow[(i & 3) * 128 + row] = er;
+      tc::tmem_st_wait();
+      tc::fence_before_sync();
+      tc::mbar_arrive(s.empty + j);
+      tc::mbar_arrive(s.afull + j);
+      tc::mbar_arrive(s.eready + (i & 3));
+    }
   } else {
-    // ---------------- workers: two ping-pong groups of 8 warps (warps 2-9, 10-17) -------
-    // group g handles local tiles i = g, g+2, ...; a row is shared by two warps of the
-    // same TMEM lane quarter (warp % 4): half hf owns K-columns / output columns
-    // [hf*X/2, (hf+1)*X/2).  Row-wide quantities (scale, softmax max/sum, p, q) are
-    // combined through smem with a 256-thread named barrier per group.
-    const int wi = warp - 2;
+    // ---------------- epilogue: two groups of 8 warps (6-13, 14-21) -----------------
+    // group g handles tiles i = g, g+2, ... from ACC[g]; a row is shared by two warps of
+    // the same TMEM lane quarter: half hf owns output columns [hf*D/2, (hf+1)*D/2).
+    const int wi = warp - 6;
     const int g = wi >> 3;
     const int hf = (wi >> 2) & 1;
     const int qd = warp & 3;
@@ -299,67 +331,22 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
     const uint32_t lane_base = tmem + (uint32_t(qd * 32) << 16);
     float *xg = s.xch + g * (2 * 2 * 128);           // [value][half][row]
     float *wbuf = s.xbuf + wi * (8 * 36);
-    const int KH = Kpad / 2;                          // K-elements per half (Kpad = 64 or 128)
+    constexpr int DH = D / 2;
+    const int cb = hf * DH;
     for (int i = g; i < my; i += 2) {
       const int j = i & 1;
-      const uint32_t par = (i >> 1) & 1;
       const long r0 = long(blockIdx.x + i * gridDim.x) * TM;
       const int nrows = min(TM, int(a.R - r0));
       const bool live = row < nrows;
-      int sidx = 0, didx = 0;
-      if (EPI == EPI_EDGE && live && hf == 0) {
-        sidx = __ldg(a.src + r0 + row);
-        didx = __ldg(a.dst + r0 + row);
-      }
-      // -- convert this thread's half row into TMEM A[j]
-      TRACE(2 + warp, i, 0);
-      tc::mbar_wait(s.full + j, par);
-      TRACE(2 + warp, i, 1);
-      const float *sl = s.slot(j);
-      const int kb = hf * KH, ke = min(K, kb + KH);
-      float mx = 0.f;
-      if (live)
-#pragma unroll 4
-        for (int k = kb; k < ke; k += 4) {
-          const float4 v = slot_ld4(sl, row, k);
-          mx = fmaxf(mx, fmaxf(fmaxf(fabsf(v.x), fabsf(v.y)), fmaxf(fabsf(v.z), fabsf(v.w))));
-        }
-      xg[hf * 128 + row] = mx;
-      group_bar(g);
-      mx = fmaxf(mx, xg[(hf ^ 1) * 128 + row]);
-      const int er = scale_exp(mx);
-      const float xs = ldexpf(1.f, er);
-      for (int c0 = 0; c0 < KH / 2; c0 += 32) {       // TMEM columns of this half
-        uint32_t x0[32], x1[32];
-#pragma unroll
-        for (int u = 0; u < 32; u += 2) {
-          const int k = kb + 2 * (c0 + u);
-          float4 v = make_float4(0.f, 0.f, 0.f, 0.f);
-          if (live && k < K) v = slot_ld4(sl, row, k);
-          split2(v.x * xs, v.y * xs, x0[u], x1[u]);
-          split2(v.z * xs, v.w * xs, x0[u + 1], x1[u + 1]);
-        }
-        const uint32_t col = a_col(j) + uint32_t(kb / 2 + c0);
-        tc::tmem_st32(lane_base + col, x0);
-        tc::tmem_st32(lane_base + col + Kpad / 2, x1);
-      }
-      tc::tmem_st_wait();
-      tc::fence_before_sync();
-      tc::mbar_arrive(s.empty + j);
-      tc::mbar_arrive(s.afull + j);
       float aux = 0.f;
-      if (EPI == EPI_EDGE) {                          // α = p[s] + q[t] (R1), exchanged
-        if (hf == 0) {
-          aux = live ? __ldg(a.pin + sidx) + __ldg(a.qin + didx) : 0.f;
-          xg[row] = aux;
-        }
-      }
-      // -- epilogue over output columns [hf*D/2, (hf+1)*D/2)
-      TRACE(2 + warp, i, 2);
-      tc::mbar_wait(s.accfull + j, par);
-      TRACE(2 + warp, i, 3);
+      if (EPI == EPI_EDGE && hf == 0 && live)
+        aux = __ldg(a.pin + __ldg(a.src + r0 + row)) + __ldg(a.qin + __ldg(a.dst + r0 + row));  // α (R1)
+      tc::mbar_wait(s.eready + (i & 3), (i >> 2) & 1);
+      const int er = s.erow[(i & 3) * 128 + row];
+      tc::mbar_wait(s.accfull + j, (i >> 1) & 1);
       tc::fence_after_sync();
       if (EPI == EPI_EDGE) {
+        if (hf == 0) xg[row] = aux;
         group_bar(g);
         aux = xg[row];
       }
@@ -367,29 +354,28 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
       const long grow = r0 + row;
       const long wrow0 = r0 + qd * 32;
       const int wrows = max(0, min(32, nrows - qd * 32));
-      constexpr int DH = D / 2;
-      const int cb = hf * DH;
+      const uint32_t acc = lane_base + acc_col(j) + cb;
       if (EPI == EPI_GATE) {
-        float v[DH];
+        float m = -INFINITY;
 #pragma unroll
         for (int c0 = 0; c0 < DH; c0 += 32) {
           uint32_t r[32];
-          tc::tmem_ld32(lane_base + acc_col(j) + cb + c0, r);
+          tc::tmem_ld32(acc + c0, r);
           tc::tmem_ld_wait();
 #pragma unroll
-          for (int u = 0; u < 32; ++u) v[c0 + u] = __uint_as_float(r[u]) * un;
+          for (int u = 0; u < 32; ++u) m = fmaxf(m, __uint_as_float(r[u]) * un);
         }
-        float m = -INFINITY;
-#pragma unroll
-        for (int c = 0; c < DH; ++c) m = fmaxf(m, v[c]);
         xg[hf * 128 + row] = m;
         group_bar(g);
         m = fmaxf(m, xg[(hf ^ 1) * 128 + row]);
         float sum = 0.f;
 #pragma unroll
-        for (int c = 0; c < DH; ++c) {
-          v[c] = fast_exp(v[c] - m);
-          sum += v[c];
+        for (int c0 = 0; c0 < DH; c0 += 32) {
+          uint32_t r[32];
+          tc::tmem_ld32(acc + c0, r);
+          tc::tmem_ld_wait();
+#pragma unroll
+          for (int u = 0; u < 32; ++u) sum += fast_exp(__uint_as_float(r[u]) * un - m);
         }
         xg[256 + hf * 128 + row] = sum;
         group_bar(g);
@@ -397,9 +383,12 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
         const float inv = fast_rcp(sum);
 #pragma unroll
         for (int c0 = 0; c0 < DH; c0 += 32) {
+          uint32_t r[32];
+          tc::tmem_ld32(acc + c0, r);
+          tc::tmem_ld_wait();
           float o[32];
 #pragma unroll
-          for (int u = 0; u < 32; ++u) o[u] = v[c0 + u] * inv;
+          for (int u = 0; u < 32; ++u) o[u] = fast_exp(__uint_as_float(r[u]) * un - m) * inv;
           warp_store_chunk<D>(wbuf, a.out, wrow0, wrows, cb + c0, o, lane);
         }
       } else {
@@ -407,7 +396,7 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
 #pragma unroll
         for (int c0 = 0; c0 < DH; c0 += 32) {
           uint32_t r[32];
-          tc::tmem_ld32(lane_base + acc_col(j) + cb + c0, r);
+          tc::tmem_ld32(acc + c0, r);
           tc::tmem_ld_wait();
           float o[32];
 #pragma unroll
@@ -441,8 +430,8 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
           }
         }
       }
-      TRACE(2 + warp, i, 4);
       tc::fence_before_sync();
+      tc::mbar_arrive(s.accfree + j);
       group_bar(g);        // the exchange buffer is reused by the next tile
     }
   }
@@ -606,16 +595,3 @@ int launch_forward_layer_tc(const occu_ctx *ctx, const DevCsr &csr, const FwdLay
 
 }  // namespace occu
 
-#ifdef OCCU_TC_TRACE
-extern "C" int occu_debug_trace(long long *host, int max_events) {
-  int n = 0;
-  cudaDeviceSynchronize();
-  cudaMemcpyFromSymbol(&n, occu::g_trace_n, sizeof(int));
-  n = n < max_events ? n : max_events;
-  n = n < 4096 ? n : 4096;
-  cudaMemcpyFromSymbol(host, occu::g_trace, size_t(n) * 4 * sizeof(long long));
-  const int zero = 0;
-  cudaMemcpyToSymbol(occu::g_trace_n, &zero, sizeof(int));
-  return n;
-}
-#endif
