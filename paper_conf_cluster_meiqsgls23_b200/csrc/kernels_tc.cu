@@ -92,7 +92,7 @@ __host__ __device__ inline int nbox_of(int K) { return (K + 31) / 32; }
 __host__ __device__ inline size_t smem_bytes(int D, int K) {
   const size_t img = size_t(kpad_of(K)) * D * 2;
   const size_t slot = size_t(nbox_of(K)) * 16384;
-  return 1024 + 2 * img + 2 * slot + 4096 + 16 * 8 * 36 * 4 + 2 * 2 * 2 * 128 * 4;
+  return 1024 + 2 * img + 2 * slot + 4096 + 16 * 16 * 20 * 4 + 2 * 2 * 2 * 128 * 4;
 }
 
 __device__ __forceinline__ Smem carve(uint8_t *raw, int D, int K) {
@@ -120,7 +120,7 @@ __device__ __forceinline__ Smem carve(uint8_t *raw, int D, int K) {
   s.avec = reinterpret_cast<float *>(misc + 512);
   s.erow = reinterpret_cast<int *>(misc + 1536);
   s.xbuf = reinterpret_cast<float *>(misc + 4096);
-  s.xch = s.xbuf + 16 * 8 * 36;
+  s.xch = s.xbuf + 16 * 16 * 20;
   return s;
 }
 
@@ -146,23 +146,24 @@ __device__ __forceinline__ void split2(float v0, float v1, uint32_t &hi, uint32_
 // instruction writes 4 full 128-byte lines instead of 32 partial ones.
 template <int D>
 __device__ __forceinline__ void warp_store_chunk(float *buf, float *__restrict__ out, long wrow0,
-                                                 int wrows, int c0, const float (&v)[32], int lane) {
+                                                 int wrows, int c0, const float (&v)[16], int lane) {
+  // 16 columns (64 B) per row; two 16-row passes through a 16 x 20 buffer
 #pragma unroll
-  for (int h = 0; h < 4; ++h) {
-    if ((lane >> 3) == h) {
-      float *b = buf + (lane & 7) * 36;
+  for (int h = 0; h < 2; ++h) {
+    if ((lane >> 4) == h) {
+      float *b = buf + (lane & 15) * 20;
 #pragma unroll
-      for (int u = 0; u < 32; u += 4)
+      for (int u = 0; u < 16; u += 4)
         *reinterpret_cast<float4 *>(b + u) = make_float4(v[u], v[u + 1], v[u + 2], v[u + 3]);
     }
     __syncwarp();
 #pragma unroll
     for (int it = 0; it < 2; ++it) {
-      const int idx = it * 32 + lane, r = idx >> 3, c4 = (idx & 7) * 4;
-      const int rr = h * 8 + r;
+      const int idx = it * 32 + lane, r = idx >> 2, c4 = (idx & 3) * 4;
+      const int rr = h * 16 + r;
       if (rr < wrows)
         *reinterpret_cast<float4 *>(out + (wrow0 + rr) * D + c0 + c4) =
-            *reinterpret_cast<const float4 *>(buf + r * 36 + c4);
+            *reinterpret_cast<const float4 *>(buf + r * 20 + c4);
     }
     __syncwarp();
   }
@@ -299,18 +300,18 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
         }
       const int er = scale_exp(mx);
       const float xs = ldexpf(1.f, er);
-      for (int c0 = 0; c0 < Kpad / 2; c0 += 32) {
-        uint32_t x0[32], x1[32];
+      for (int c0 = 0; c0 < Kpad / 2; c0 += 16) {
+        uint32_t x0[16], x1[16];
 #pragma unroll
-        for (int u = 0; u < 32; u += 2) {
+        for (int u = 0; u < 16; u += 2) {
           const int k = 2 * (c0 + u);
           float4 v = make_float4(0.f, 0.f, 0.f, 0.f);
           if (live && k < K) v = slot_ld4(sl, row, k);
           split2(v.x * xs, v.y * xs, x0[u], x1[u]);
           split2(v.z * xs, v.w * xs, x0[u + 1], x1[u + 1]);
         }
-        tc::tmem_st32(lane_base + a_col(j) + c0, x0);
-        tc::tmem_st32(lane_base + a_col(j) + Kpad / 2 + c0, x1);
+        tc::tmem_st16(lane_base + a_col(j) + c0, x0);
+        tc::tmem_st16(lane_base + a_col(j) + Kpad / 2 + c0, x1);
       }
       s.erow[(i & 3) * 128 + row] = er;
       tc::tmem_st_wait();
@@ -330,7 +331,7 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
     const int row = qd * 32 + lane;
     const uint32_t lane_base = tmem + (uint32_t(qd * 32) << 16);
     float *xg = s.xch + g * (2 * 2 * 128);           // [value][half][row]
-    float *wbuf = s.xbuf + wi * (8 * 36);
+    float *wbuf = s.xbuf + wi * (16 * 20);
     constexpr int DH = D / 2;
     const int cb = hf * DH;
     for (int i = g; i < my; i += 2) {
@@ -358,49 +359,49 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
       if (EPI == EPI_GATE) {
         float m = -INFINITY;
 #pragma unroll
-        for (int c0 = 0; c0 < DH; c0 += 32) {
-          uint32_t r[32];
-          tc::tmem_ld32(acc + c0, r);
+        for (int c0 = 0; c0 < DH; c0 += 16) {
+          uint32_t r[16];
+          tc::tmem_ld16(acc + c0, r);
           tc::tmem_ld_wait();
 #pragma unroll
-          for (int u = 0; u < 32; ++u) m = fmaxf(m, __uint_as_float(r[u]) * un);
+          for (int u = 0; u < 16; ++u) m = fmaxf(m, __uint_as_float(r[u]) * un);
         }
         xg[hf * 128 + row] = m;
         group_bar(g);
         m = fmaxf(m, xg[(hf ^ 1) * 128 + row]);
         float sum = 0.f;
 #pragma unroll
-        for (int c0 = 0; c0 < DH; c0 += 32) {
-          uint32_t r[32];
-          tc::tmem_ld32(acc + c0, r);
+        for (int c0 = 0; c0 < DH; c0 += 16) {
+          uint32_t r[16];
+          tc::tmem_ld16(acc + c0, r);
           tc::tmem_ld_wait();
 #pragma unroll
-          for (int u = 0; u < 32; ++u) sum += fast_exp(__uint_as_float(r[u]) * un - m);
+          for (int u = 0; u < 16; ++u) sum += fast_exp(__uint_as_float(r[u]) * un - m);
         }
         xg[256 + hf * 128 + row] = sum;
         group_bar(g);
         sum = hf == 0 ? sum + xg[256 + 128 + row] : xg[256 + row] + sum;   // fixed order
         const float inv = fast_rcp(sum);
-#pragma unroll
-        for (int c0 = 0; c0 < DH; c0 += 32) {
-          uint32_t r[32];
-          tc::tmem_ld32(acc + c0, r);
+#pragma unroll 1
+        for (int c0 = 0; c0 < DH; c0 += 16) {
+          uint32_t r[16];
+          tc::tmem_ld16(acc + c0, r);
           tc::tmem_ld_wait();
-          float o[32];
+          float o[16];
 #pragma unroll
-          for (int u = 0; u < 32; ++u) o[u] = fast_exp(__uint_as_float(r[u]) * un - m) * inv;
+          for (int u = 0; u < 16; ++u) o[u] = fast_exp(__uint_as_float(r[u]) * un - m) * inv;
           warp_store_chunk<D>(wbuf, a.out, wrow0, wrows, cb + c0, o, lane);
         }
       } else {
         float pp = 0.f, qq = 0.f;
-#pragma unroll
-        for (int c0 = 0; c0 < DH; c0 += 32) {
-          uint32_t r[32];
-          tc::tmem_ld32(acc + c0, r);
+#pragma unroll 1
+        for (int c0 = 0; c0 < DH; c0 += 16) {
+          uint32_t r[16];
+          tc::tmem_ld16(acc + c0, r);
           tc::tmem_ld_wait();
-          float o[32];
+          float o[16];
 #pragma unroll
-          for (int u = 0; u < 32; u += 4) {
+          for (int u = 0; u < 16; u += 4) {
             if (EPI == EPI_NODE) {
               const float4 as4 = *reinterpret_cast<const float4 *>(s.avec + cb + c0 + u);
               const float4 ad4 = *reinterpret_cast<const float4 *>(s.avec + D + cb + c0 + u);
