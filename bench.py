@@ -105,19 +105,36 @@ def dist_env():
 
 
 # ---------------------------------------------------------------- algorithmic bytes
+# Bytes each kernel must move per step (all its launches), fp32 storage, d = 128,
+# with perfect reuse of gathered rows (each h̄ / p / q row counted once).  DESIGN.md §6.
+def algorithmic_bytes(N, E, B, d=128, F_n=80, F_e=4, L=3):
+    s = 4
+    node = s * N * F_n + s * N * d * (L - 1) + s * N * (d + 2) * L                # read h_in, write h̄,p,q
+    edge_small = s * E * F_e + 8 * E + 8 * N + s * E * d                          # layer 1
+    edge_tc = (L - 1) * (s * E * d + 8 * E + 8 * N + s * E * d)                    # layers 2..L
+    gate = L * (s * E * d + s * E * d)                                             # read e', write g
+    gather = L * (s * E * d + s * N * d + 4 * E + 4 * (N + 1) + s * N * d)         # g, h̄, idx, h
+    readout = s * N * d + s * B * (2 * d + 1)
+    permute = s * E * F_e * 2 + 4 * E
+    return {"node_tc": node, "edge_small": edge_small, "edge_tc": edge_tc, "gate_tc": gate,
+            "gather_segsum": gather, "readout_head": readout, "permute_e0": permute,
+            # SIMT path kernels
+            "node_gemm": node, "edge_fwd": edge_small + edge_tc + gate}
+
+
 def aggregation_bytes(N, E, d, s=4):
-    """a5 + a6 (gather_segsum): read g [E,d], gather h̄[src] once per node (perfect
-    L2 reuse), write h [N,d], read in_src/in_ptr."""
+    """a5 + a6 per launch (gather_segsum): read g [E,d], gather h̄[src] once per node,
+    read in_src / in_ptr, write h [N,d]."""
     return s * (E * d + N * d + N * d) + 4 * (E + N + 1)
 
 
-def edge_fwd_flops(E, d, de_in):
-    """a3 + a4: two GEMMs per edge (W_e: 2·de_in·d, W_m: 2·d·d)."""
-    return 2.0 * E * d * (de_in + d)
-
-
-def node_gemm_flops(N, d, d_in):
-    return 2.0 * N * d * d_in
+def load_traffic():
+    """Per-launch DRAM bytes (ncu dram__bytes_read+write) committed under profiles/."""
+    try:
+        with open(os.path.join(ROOT, "profiles", "traffic.json")) as f:
+            return json.load(f)
+    except Exception:
+        return {}
 
 
 def cpu_cores_used():
@@ -284,43 +301,41 @@ def main():
     ms_step = max_over_ranks(float(np.sum(times)) / args.steps)
     value = B * world / (ms_step * 1e-3)
 
-    # roofline: per-kernel device time inside the timed region (CUDA events)
+    # roofline: per-kernel device time inside the timed region (CUDA events on the
+    # library's launch stream), algorithmic bytes per kernel
     d = 128
-    tot_kernel = sum(v[0] for v in prof.values())
-    shares = {k: v[0] / max(tot_kernel, 1e-9) for k, v in prof.items()}
-    dom = max(prof, key=lambda k: prof[k][0])
-
-    def kernel_avg_ms(name):
-        t, n = prof.get(name, (0.0, 0))
-        return t / max(n, 1)
-
-    agg_bytes_per_launch = aggregation_bytes(N, E, d)
-    agg_ms = kernel_avg_ms("gather_segsum")
-    agg = {"kernel": "gather_segsum", "bound": "hbm",
-           "achieved": agg_bytes_per_launch / (agg_ms * 1e-3) / 1e9 if agg_ms else None,
-           "peak": peaks["hbm_gbs"], "unit": "GB/s",
-           "algorithmic_bytes_per_launch": agg_bytes_per_launch, "avg_ms": agg_ms}
+    alg = algorithmic_bytes(N, E, B, d)
+    traffic = load_traffic()
+    kernels = {}
+    for k, (ms_tot, n) in prof.items():
+        ms = ms_tot / args.steps
+        by = alg.get(k)
+        gbs = by / (ms * 1e-3) / 1e9 if (by and ms > 0) else None
+        kernels[k] = {"ms_per_step": ms, "launches_per_step": n / args.steps,
+                      "algorithmic_bytes_per_step": by, "achieved_GBps": gbs,
+                      "frac_of_measured_hbm": gbs / peaks["hbm_gbs"] if gbs else None}
+    dom = max(kernels, key=lambda k: kernels[k]["ms_per_step"])
+    tot_kernel = sum(v["ms_per_step"] for v in kernels.values())
+    kd = kernels[dom]
+    lpl = max(kd["launches_per_step"], 1)
+    tr = traffic.get(dom)
+    roof = {"kernel": dom, "bound": "hbm", "achieved": kd["achieved_GBps"], "peak": peaks["hbm_gbs"],
+            "unit": "GB/s", "frac": kd["frac_of_measured_hbm"],
+            "traffic": tr.get("dram_bytes_per_launch") if tr else None,
+            "algorithmic_bytes_per_launch": (kd["algorithmic_bytes_per_step"] or 0) / lpl,
+            "avg_launch_ms": kd["ms_per_step"] / lpl, "peak_kind": peak_src,
+            "share_of_step": kd["ms_per_step"] / tot_kernel if tot_kernel else None}
+    agg_ms = kernels.get("gather_segsum", {}).get("ms_per_step")
+    agg_launch = agg_ms / 3 if agg_ms else None
+    agg_b = aggregation_bytes(N, E, d)
+    agg = {"kernel": "gather_segsum", "bound": "hbm", "algorithmic_bytes_per_launch": agg_b,
+           "avg_ms": agg_launch,
+           "achieved": agg_b / (agg_launch * 1e-3) / 1e9 if agg_launch else None,
+           "peak": peaks["hbm_gbs"], "unit": "GB/s"}
     agg["frac"] = agg["achieved"] / agg["peak"] if agg["achieved"] else None
     agg["frac_of_8TBps"] = agg["achieved"] / 8000.0 if agg["achieved"] else None
-    # FP32 SIMT GEMM kernels are FP32-ALU bound: peak = 148 SMs x 128 FMA/clk x 2 x max clock
-    alu_peak_tflops = 148 * 128 * 2 * peaks.get("sm_max_mhz", 1965.0) * 1e6 / 1e12
-    if dom == "edge_fwd":
-        # per launch: layer 1 (de_in = 4) and layers 2-3 (de_in = d): average over the 3 launches
-        fl = (edge_fwd_flops(E, d, 4) + 2 * edge_fwd_flops(E, d, d)) / 3
-        roof = {"kernel": dom, "bound": "alu", "achieved": fl / (kernel_avg_ms(dom) * 1e-3) / 1e12,
-                "peak": alu_peak_tflops, "unit": "TFLOP/s", "traffic": None,
-                "peak_source": "DESIGN.md §6: 148 SM x 128 FP32 lanes x 2 x 1965 MHz"}
-    elif dom == "node_gemm":
-        fl = (node_gemm_flops(N, d, 80) + 2 * node_gemm_flops(N, d, d)) / 3
-        roof = {"kernel": dom, "bound": "alu", "achieved": fl / (kernel_avg_ms(dom) * 1e-3) / 1e12,
-                "peak": alu_peak_tflops, "unit": "TFLOP/s", "traffic": None,
-                "peak_source": "DESIGN.md §6: 148 SM x 128 FP32 lanes x 2 x 1965 MHz"}
-    else:
-        roof = {"kernel": "gather_segsum", "bound": "hbm", "achieved": agg["achieved"],
-                "peak": peaks["hbm_gbs"], "unit": "GB/s", "traffic": None}
-    roof["frac"] = roof["achieved"] / roof["peak"] if roof["achieved"] else None
-    roof["peak_kind"] = peak_src
-    roof["share_of_step"] = shares.get(roof["kernel"])
+    if traffic.get("gather_segsum"):
+        agg["traffic"] = traffic["gather_segsum"].get("dram_bytes_per_launch")
 
     # ---- e2e through the public API with host buffers (pinned), pack included
     pin_nf = torch.from_numpy(batch.node_feat).pin_memory()
@@ -386,7 +401,8 @@ def main():
             "clocks": clk.summary(),
             "roofline": roof,
             "aggregation": agg,
-            "kernel_ms_per_step": {k: v[0] / args.steps for k, v in prof.items()},
+            "kernel_ms_per_step": {k: v["ms_per_step"] for k, v in kernels.items()},
+            "kernels": kernels,
             "e2e": e2e,
             "train": train,
             "cpu_baseline": cpu,

@@ -1,0 +1,12 @@
+#!/bin/bash
+# Round profiling (one GPU): launch list of the bench command + ncu --set full of
+# the hot kernels; summarised into profiles/ by scripts/summarize_ncu.py (run here).
+cd "${GRAFT_REPO_ROOT:-/root/repo}"; mkdir -p gpurun_out
+timeout 900 ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum \
+  --clock-control none -c 400 --csv --log-file gpurun_out/launches.csv \
+  python bench.py --steps 3 --warmup 3 --no-cpu > gpurun_out/launches_bench.log 2>&1
+echo "launches rc=$?" >> gpurun_out/launches_bench.log
+timeout 900 ncu --set full --clock-control none --import-source on \
+  -k regex:"rowgemm|gather_segsum|edge_small" -s 7 -c 7 -o gpurun_out/prof_full \
+  python scripts/prof_driver.py --steps 2 > gpurun_out/prof_full.log 2>&1
+echo "full rc=$?" >> gpurun_out/prof_full.log
