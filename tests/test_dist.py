@@ -1,0 +1,73 @@
+"""Data-parallel host logic on CPU: LPT sharding, contiguous inference ranges,
+and a world_size-2 gloo run checking that per-rank gradients of the LPT shards
+(loss scaled by the GLOBAL batch, R15), summed by a real allreduce, equal the
+full-batch gradient.  (The GPU path uses the same shards with NCCL inside the
+library.)"""
+import os
+
+import numpy as np
+import pytest
+
+from occu_gen import configs
+from paper_conf_cluster_meiqsgls23_b200 import dist
+
+
+def test_lpt_shard_covers_and_balances():
+    b = configs.mixture(60, 1004)
+    w = dist.graph_work(b.graphs)
+    for world in (1, 2, 3, 8):
+        sh = dist.lpt_shard(w, world)
+        flat = sorted(i for s in sh for i in s)
+        assert flat == list(range(len(w)))
+        loads = [int(w[s].sum()) for s in sh]
+        assert max(loads) - min(loads) <= int(w.max())          # LPT bound
+        assert sh == dist.lpt_shard(w, world)                   # deterministic
+        assert all(s == sorted(s) for s in sh)
+
+
+def test_contiguous_shard():
+    w = np.array([5, 1, 1, 1, 8, 2, 2, 3, 9, 1])
+    for world in (1, 2, 4):
+        rg = dist.contiguous_shard(w, world)
+        assert rg[0][0] == 0 and rg[-1][1] == len(w)
+        assert all(rg[r][1] == rg[r + 1][0] for r in range(world - 1))
+
+
+def _worker(rank, world, port, q):
+    import torch
+    import torch.distributed as tdist
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    tdist.init_process_group("gloo", rank=rank, world_size=world)
+    import oracle
+    b = configs.random_dag_batch(12, 77, max_nodes=15, hub=True)
+    cfg = dict(L=2, F_n=80, F_e=4, d=8, d_h=8, aggr=0, msg=0, slope=0.01)
+    from occu_gen import weights
+    params = oracle.unflatten(cfg, weights.init_flat(weights.ModelConfig(L=2, d=8, d_h=8), 3).astype(np.float64))
+    idx = dist.lpt_shard(dist.graph_work(b.graphs), world)[rank]
+    loc = b.subset(idx)
+    loss, g = oracle.loss_and_grads(params, cfg, loc.graphs, loc.node_feat, loc.edge_feat,
+                                    loc.targets, global_batch=b.num_graphs)
+    flat = torch.tensor(np.concatenate([np.ravel(g[k]) for k, _ in oracle.param_shapes(cfg)] + [[loss]]))
+    tdist.all_reduce(flat)
+    if rank == 0:
+        lf, gf = oracle.loss_and_grads(params, cfg, b.graphs, b.node_feat, b.edge_feat, b.targets)
+        ref = np.concatenate([np.ravel(gf[k]) for k, _ in oracle.param_shapes(cfg)] + [[lf]])
+        q.put(float(np.max(np.abs(flat.numpy() - ref)) / np.max(np.abs(ref))))
+    tdist.barrier()
+    tdist.destroy_process_group()
+
+
+def test_dp_gloo_world2_matches_full_batch():
+    import torch.multiprocessing as mp
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = 29500 + (os.getpid() % 1000)
+    procs = [ctx.Process(target=_worker, args=(r, 2, port, q)) for r in range(2)]
+    for p in procs:
+        p.start()
+    for p in procs:
+        p.join(120)
+    assert all(p.exitcode == 0 for p in procs)
+    err = q.get(timeout=5)
+    assert err < 1e-12, err
