@@ -271,41 +271,77 @@ __global__ void __launch_bounds__(NT) gather_segsum_kernel(
     const float *__restrict__ g, const float *__restrict__ hbar,
     const int32_t *__restrict__ in_ptr, const int32_t *__restrict__ in_src, int N, int mean,
     float slope, float *__restrict__ h_out) {
+  // A warp owns NPW consecutive destination nodes, i.e. the contiguous in-CSR edge
+  // range [in_ptr[t0], in_ptr[t0+NPW]); edges are consumed in ascending order, four
+  // gathered rows in flight at a time, and each node's sum is flushed when the edge
+  // index crosses its segment end (fixed order: identical to a per-node loop).
   constexpr int V = D / 32;
+  constexpr int NPW = 8;
   const int lane = threadIdx.x & 31;
-  const int warps = (gridDim.x * NT) / 32;
-  for (int t = (blockIdx.x * NT + threadIdx.x) / 32; t < N; t += warps) {
-    const int beg = in_ptr[t], end = in_ptr[t + 1];
+  const long warps = (long(gridDim.x) * NT) / 32;
+  for (long t0 = (blockIdx.x * long(NT) + threadIdx.x) / 32 * NPW; t0 < N; t0 += warps * NPW) {
+    const int nn = int(min(long(NPW), N - t0));
+    const int ptr_l = lane <= nn ? in_ptr[t0 + lane] : 0;      // in_ptr[t0 .. t0+nn]
+    const int e_beg = __shfl_sync(0xffffffffu, ptr_l, 0);
+    const int e_end = __shfl_sync(0xffffffffu, ptr_l, nn);
+    int node = 0;                                               // local node index
+    int seg_end = __shfl_sync(0xffffffffu, ptr_l, 1);
     float acc[V];
 #pragma unroll
     for (int c = 0; c < V; ++c) acc[c] = 0.f;
-    for (int base = beg; base < end; base += 32) {
-      const int cnt = min(32, end - base);
+#define OCCU_FLUSH_NODE(nd)                                                                  \
+  do {                                                                                       \
+    const int deg_ = __shfl_sync(0xffffffffu, ptr_l, (nd) + 1) - __shfl_sync(0xffffffffu, ptr_l, (nd)); \
+    float *o_ = h_out + (t0 + (nd)) * D + lane * V;                                          \
+    _Pragma("unroll") for (int c = 0; c < V; ++c) {                                          \
+      float a_ = acc[c];                                                                     \
+      if (mean) a_ = a_ / float(deg_ > 0 ? deg_ : 1);                                        \
+      o_[c] = lrelu(a_, slope);                                                              \
+      acc[c] = 0.f;                                                                          \
+    }                                                                                        \
+  } while (0)
+    for (int base = e_beg; base < e_end; base += 32) {
+      const int cnt = min(32, e_end - base);
       const int s_l = lane < cnt ? in_src[base + lane] : 0;
-      for (int j = 0; j < cnt; ++j) {
-        const int s = __shfl_sync(0xffffffffu, s_l, j);
-        const float *gr = g + long(base + j) * D + lane * V;
-        const float *hr = hbar + long(s) * D + lane * V;
-        if (V == 4) {
-          const float4 a = __ldg(reinterpret_cast<const float4 *>(gr));
-          const float4 b = __ldg(reinterpret_cast<const float4 *>(hr));
-          acc[0] = fmaf(a.x, b.x, acc[0]);
-          acc[1 % V] = fmaf(a.y, b.y, acc[1 % V]);
-          acc[2 % V] = fmaf(a.z, b.z, acc[2 % V]);
-          acc[3 % V] = fmaf(a.w, b.w, acc[3 % V]);
-        } else {
+      for (int j = 0; j < cnt; j += 4) {
+        float gv[4][V], hv[4][V];
 #pragma unroll
-          for (int c = 0; c < V; ++c) acc[c] = fmaf(__ldg(gr + c), __ldg(hr + c), acc[c]);
+        for (int u = 0; u < 4; ++u) {
+          const int s = __shfl_sync(0xffffffffu, s_l, (j + u) & 31);
+          if (j + u < cnt) {
+            const float *gr = g + long(base + j + u) * D + lane * V;
+            const float *hr = hbar + long(s) * D + lane * V;
+            if (V == 4) {
+              const float4 a = __ldg(reinterpret_cast<const float4 *>(gr));
+              const float4 b2 = __ldg(reinterpret_cast<const float4 *>(hr));
+              gv[u][0] = a.x; gv[u][1 % V] = a.y; gv[u][2 % V] = a.z; gv[u][3 % V] = a.w;
+              hv[u][0] = b2.x; hv[u][1 % V] = b2.y; hv[u][2 % V] = b2.z; hv[u][3 % V] = b2.w;
+            } else {
+#pragma unroll
+              for (int c = 0; c < V; ++c) {
+                gv[u][c] = __ldg(gr + c);
+                hv[u][c] = __ldg(hr + c);
+              }
+            }
+          }
+        }
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+          if (j + u < cnt) {
+            const int k = base + j + u;
+            while (k >= seg_end) {                  // warp-uniform
+              OCCU_FLUSH_NODE(node);
+              ++node;
+              seg_end = __shfl_sync(0xffffffffu, ptr_l, node + 1);
+            }
+#pragma unroll
+            for (int c = 0; c < V; ++c) acc[c] = fmaf(gv[u][c], hv[u][c], acc[c]);
+          }
         }
       }
     }
-    const int deg = end - beg;
-#pragma unroll
-    for (int c = 0; c < V; ++c) {
-      float a = acc[c];
-      if (mean) a = a / float(deg > 0 ? deg : 1);
-      h_out[long(t) * D + lane * V + c] = lrelu(a, slope);
-    }
+    for (; node < nn; ++node) OCCU_FLUSH_NODE(node);   // remaining (and in-degree-0) nodes
+#undef OCCU_FLUSH_NODE
   }
 }
 
@@ -794,7 +830,7 @@ static int forward_layer_impl(const occu_ctx *ctx, const DevCsr &csr, const FwdL
   }
   if (csr.N > 0) {
     OCCU_PROF_BEGIN(ctx, "gather_segsum", st);
-    gather_segsum_kernel<D><<<grid_for(long(csr.N) * 32, NT, 16 * sms), NT, 0, st>>>(
+    gather_segsum_kernel<D><<<grid_for(long(csr.N) * 4, NT, 16 * sms), NT, 0, st>>>(
         a.g, a.hbar, csr.in_ptr, csr.in_src, csr.N, ctx->cfg.aggr == OCCU_AGGR_MEAN,
         ctx->cfg.slope, a.h_out);
     OCCU_PROF_END(ctx);
@@ -809,7 +845,7 @@ static int gather_impl(const occu_ctx *ctx, const DevCsr &csr, const float *g, c
                        float *h_out, cudaStream_t st) {
   if (csr.N <= 0) return 0;
   OCCU_PROF_BEGIN(ctx, "gather_segsum", st);
-  gather_segsum_kernel<D><<<grid_for(long(csr.N) * 32, NT, 16 * ctx->num_sms), NT, 0, st>>>(
+  gather_segsum_kernel<D><<<grid_for(long(csr.N) * 4, NT, 16 * ctx->num_sms), NT, 0, st>>>(
       g, hbar, csr.in_ptr, csr.in_src, csr.N, ctx->cfg.aggr == OCCU_AGGR_MEAN, ctx->cfg.slope,
       h_out);
   OCCU_PROF_END(ctx);

@@ -444,39 +444,51 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
 
 // Layer-1 edge transform (F_e small, e.g. 4): e' = σ(α · W_e e) on CUDA cores,
 // one warp per edge, lanes over 4-channel groups (coalesced 512-byte rows).
-template <int D>
+template <int D, int KM>
 __global__ void __launch_bounds__(256) edge_small_kernel(
     const float *__restrict__ e_in, int Ke, const float *__restrict__ W_e,
     const float *__restrict__ p, const float *__restrict__ q, const int32_t *__restrict__ in_src,
     const int32_t *__restrict__ in_dst, int E, float *__restrict__ e_out) {
+  // One warp per 4 consecutive edges (4 independent index/α chains in flight),
+  // lanes over 4-channel groups: coalesced 512-byte rows.  Ke <= 16.
   extern __shared__ float wsm[];            // [Ke][D] = W_eᵀ (conflict-free float4 reads)
   for (int i = threadIdx.x; i < D * Ke; i += blockDim.x) wsm[(i % Ke) * D + i / Ke] = W_e[i];
   __syncthreads();
-  constexpr int G = D / 4;                  // lanes per edge (4 channels each)
-  constexpr int EPW = 32 / G;               // edges per warp step
+  constexpr int G = D / 4;                  // lanes per edge row
+  constexpr int RPI = 32 / G;               // rows per warp instruction
+  constexpr int EPW = 4 * RPI;              // edges per warp iteration
   const int lane = threadIdx.x & 31;
   const int sub = lane / G, c = (lane % G) * 4;
   const long nwarps = long(gridDim.x) * (blockDim.x / 32);
-  for (long k = (blockIdx.x * long(blockDim.x / 32) + threadIdx.x / 32) * EPW + sub; k < E;
-       k += nwarps * EPW) {
-    const float al = __ldg(p + in_src[k]) + __ldg(q + in_dst[k]);
-    float e[16];
+  for (long k0 = (blockIdx.x * long(blockDim.x / 32) + threadIdx.x / 32) * EPW; k0 < E;
+       k0 += nwarps * EPW) {
+    float al[4], ev[4][KM];
 #pragma unroll
-    for (int j = 0; j < 16; ++j) e[j] = j < Ke ? __ldg(e_in + k * Ke + j) : 0.f;
-    float z[4] = {0.f, 0.f, 0.f, 0.f};
+    for (int u = 0; u < 4; ++u) {
+      const long k = k0 + u * RPI + sub;
+      al[u] = 0.f;
+      if (k < E) al[u] = __ldg(p + in_src[k]) + __ldg(q + in_dst[k]);
 #pragma unroll
-    for (int j = 0; j < 16; ++j)
-      if (j < Ke) {
-        const float4 w = *reinterpret_cast<const float4 *>(wsm + j * D + c);
-        z[0] = fmaf(w.x, e[j], z[0]);
-        z[1] = fmaf(w.y, e[j], z[1]);
-        z[2] = fmaf(w.z, e[j], z[2]);
-        z[3] = fmaf(w.w, e[j], z[3]);
-      }
-    float o[4];
+      for (int j = 0; j < KM; ++j) ev[u][j] = (j < Ke && k < E) ? __ldg(e_in + k * Ke + j) : 0.f;
+    }
 #pragma unroll
-    for (int u = 0; u < 4; ++u) o[u] = fast_rcp(1.f + fast_exp(-(al * z[u])));
-    *reinterpret_cast<float4 *>(e_out + k * D + c) = make_float4(o[0], o[1], o[2], o[3]);
+    for (int u = 0; u < 4; ++u) {
+      const long k = k0 + u * RPI + sub;
+      float z[4] = {0.f, 0.f, 0.f, 0.f};
+#pragma unroll
+      for (int j = 0; j < KM; ++j)
+        if (j < Ke) {
+          const float4 w = *reinterpret_cast<const float4 *>(wsm + j * D + c);
+          z[0] = fmaf(w.x, ev[u][j], z[0]);
+          z[1] = fmaf(w.y, ev[u][j], z[1]);
+          z[2] = fmaf(w.z, ev[u][j], z[2]);
+          z[3] = fmaf(w.w, ev[u][j], z[3]);
+        }
+      float o[4];
+#pragma unroll
+      for (int t = 0; t < 4; ++t) o[t] = fast_rcp(1.f + fast_exp(-(al[u] * z[t])));
+      if (k < E) *reinterpret_cast<float4 *>(e_out + k * D + c) = make_float4(o[0], o[1], o[2], o[3]);
+    }
   }
 }
 
@@ -556,11 +568,14 @@ static int tc_forward_layer_impl(const occu_ctx *ctx, const DevCsr &csr, const F
   if (csr.E > 0) {
     // a3: edge transform
     if (a.Ke <= 16) {
-      const int grid = int(std::min<long>((long(csr.E) * (D / 4) + 255) / 256, 8L * ctx->num_sms));
+      const int grid = int(std::min<long>((long(csr.E) * (D / 4) / 4 + 255) / 256, 8L * ctx->num_sms));
       OCCU_PROF_BEGIN(ctx, "edge_small", st);
-      edge_small_kernel<D><<<grid, 256, D * a.Ke * 4, st>>>(a.e_in, a.Ke, a.W_e, a.p, a.q,
-                                                             csr.in_src, csr.in_dst, csr.E,
-                                                             a.e_out);
+      if (a.Ke <= 4)
+        edge_small_kernel<D, 4><<<grid, 256, D * a.Ke * 4, st>>>(a.e_in, a.Ke, a.W_e, a.p, a.q,
+                                                                 csr.in_src, csr.in_dst, csr.E, a.e_out);
+      else
+        edge_small_kernel<D, 16><<<grid, 256, D * a.Ke * 4, st>>>(a.e_in, a.Ke, a.W_e, a.p, a.q,
+                                                                  csr.in_src, csr.in_dst, csr.E, a.e_out);
       OCCU_PROF_END(ctx);
       TC_CHECK();
       ++n;
