@@ -373,12 +373,14 @@ def main():
         step = lambda: model.train_step(csr, nf, ef, yt, 1e-4, global_num_graphs=gB, want_loss=False)
         timed(step, args.warmup)
         bar()
-        ttimes, tl = timed(step, args.steps)
+        ttimes, tl = timed(step, args.steps, profile=True)
         bar()
+        tprof = model.profile()
         tms = max_over_ranks(float(np.sum(ttimes)) / args.steps)
         loss = model.train_step(csr, nf, ef, yt, 1e-4, global_num_graphs=gB)
         train = {"value": gB / (tms * 1e-3), "unit": "graphs/s", "ms_per_step": tms,
                  "global_batch": gB, "gpu_launches": tl, "loss_after": loss,
+                 "kernel_ms_per_step": {k: v[0] / args.steps for k, v in tprof.items()},
                  "includes": "forward with saves, MSE, backward, "
                              + ("NCCL allreduce, " if world > 1 else "") + "Adam"}
 

@@ -906,6 +906,18 @@ static int wgrad(occu_ctx *ctx, const float *X, int A, const float *Y, int Bn, l
     cudaMemsetAsync(out, 0, n * 4, st);
     return 0;
   }
+  if (ctx->path == 0 && wgrad_tc_supported(A, Bn) && R >= 4096) {
+    const int sp = ctx->num_sms;
+    if (ctx->ws.partial.ensure(size_t(sp) * n * 4) != cudaSuccess) return -int(cudaErrorMemoryAllocation);
+    float *part = ctx->ws.partial.as<float>();
+    int r = launch_wgrad_tc(ctx, X, A, Y, Bn, R, sp, part, st);
+    if (r < 0) return r;
+    OCCU_PROF_BEGIN(ctx, "wgrad_reduce", st);
+    wgrad_reduce_kernel<<<grid_for(n, 256, 1024), 256, 0, st>>>(part, sp, n, out);
+    OCCU_PROF_END(ctx);
+    LAUNCH_CHECK();
+    return r + 1;
+  }
   if (ctx->ws.partial.ensure(size_t(splits) * n * 4) != cudaSuccess) return -int(cudaErrorMemoryAllocation);
   float *part = ctx->ws.partial.as<float>();
   OCCU_PROF_BEGIN(ctx, "wgrad_partial", st);

@@ -492,6 +492,148 @@ __global__ void __launch_bounds__(256) edge_small_kernel(
   }
 }
 
+// ---------------------------------------------------------------------------
+// Weight gradients on tensor cores: partial[split][a][b] = Σ_{r in split} X[r][a] Y[r][b]
+// (dW_m = DVᵀE', dW_e = DZᵀE_in, dW_u = dPᵀH_in; SURVEY §8(c) step BW).  3xTF32 with
+// the MMA's own tf32 truncation as the "hi" part: hi = X (raw fp32 in smem), lo =
+// X - trunc13(X) computed in smem; X and Y tiles arrive by 2D TMA (32 rows x 32 columns
+// SW128 boxes) and are consumed as MN-major operands (M = a, N = b, K = row).  Each CTA
+// owns a contiguous row range; partials are reduced in fixed split order afterwards.
+// ---------------------------------------------------------------------------
+constexpr int WG_NS = 3;                  // pipeline stages of 32 rows
+constexpr int WG_NTH = 192;               // warp0 TMA, warp1 MMA, warps 2-5 lo / epilogue
+
+__global__ void __launch_bounds__(WG_NTH, 1)
+wgrad_tc_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant__ CUtensorMap ymap,
+                int A, int Bn, long R, int splits, float *__restrict__ partial) {
+  extern __shared__ uint8_t smem_raw[];
+  const uint32_t sa = tc::smem_u32(smem_raw);
+  uint8_t *base = smem_raw + ((1024 - (sa & 1023)) & 1023);
+  // stage s: X raw (4 boxes x 4 KB), X lo, Y raw, Y lo
+  auto stage = [&](int s2) { return base + s2 * 65536; };
+  uint64_t *bars = reinterpret_cast<uint64_t *>(base + WG_NS * 65536);
+  uint64_t *full = bars, *lo_ready = bars + WG_NS, *empty = bars + 2 * WG_NS, *done = bars + 3 * WG_NS;
+  uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(bars + 3 * WG_NS + 1);
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int nbx = (A + 31) / 32, nby = (Bn + 31) / 32;
+  const int Npad = (Bn + 15) / 16 * 16;
+  // zero every box region once: boxes that TMA never writes (A or B < 128) stay zero
+  for (int i = threadIdx.x; i < WG_NS * 65536 / 16; i += WG_NTH)
+    reinterpret_cast<float4 *>(base)[i] = make_float4(0.f, 0.f, 0.f, 0.f);
+  if (threadIdx.x == 0) {
+    for (int j = 0; j < WG_NS; ++j) {
+      tc::mbar_init(full + j, 1);
+      tc::mbar_init(lo_ready + j, 128);
+      tc::mbar_init(empty + j, 1);
+    }
+    tc::mbar_init(done, 1);
+    tc::fence_mbar_init();
+  }
+  if (warp == 1) tc::tmem_alloc<128>(tmem_slot);
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+  tc::fence_before_sync();
+  __syncthreads();
+  tc::fence_after_sync();
+  const uint32_t tmem = *tmem_slot;
+  const long per = (R + splits - 1) / splits;
+  const long rb = blockIdx.x * per, re = min(R, rb + per);
+  const int nst = rb < re ? int((re - rb + 31) / 32) : 0;
+
+  if (warp == 0) {
+    if (lane == 0) {
+      tc::prefetch_tmap(&xmap);
+      tc::prefetch_tmap(&ymap);
+      for (int i = 0; i < nst; ++i) {
+        const int j = i % WG_NS;
+        if (i >= WG_NS) tc::mbar_wait(empty + j, ((i / WG_NS) - 1) & 1);
+        const int r0 = int(rb + long(i) * 32);
+        uint8_t *st = stage(j);
+        tc::mbar_arrive_expect_tx(full + j, uint32_t(nbx + nby) * 4096u);
+        for (int b = 0; b < nbx; ++b) tc::tma_load_2d(st + b * 4096, &xmap, 32 * b, r0, full + j);
+        for (int b = 0; b < nby; ++b) tc::tma_load_2d(st + 32768 + b * 4096, &ymap, 32 * b, r0, full + j);
+      }
+    }
+    __syncwarp();
+  } else if (warp == 1) {
+    const uint32_t idsc = tc::idesc(128, uint32_t(Npad), tc::FMT_TF32) | (1u << 15) | (1u << 16);
+    for (int i = 0; i < nst; ++i) {
+      const int j = i % WG_NS;
+      tc::mbar_wait(lo_ready + j, (i / WG_NS) & 1);
+      tc::fence_after_sync();
+      if (lane == 0) {
+        const uint32_t st = tc::smem_u32(stage(j));
+        for (int kg = 0; kg < 4; ++kg) {
+          const uint64_t ah = tc::sdesc_sw128_mn(st + kg * 1024, 4096);
+          const uint64_t al = tc::sdesc_sw128_mn(st + 16384 + kg * 1024, 4096);
+          const uint64_t bh = tc::sdesc_sw128_mn(st + 32768 + kg * 1024, 4096);
+          const uint64_t bl = tc::sdesc_sw128_mn(st + 49152 + kg * 1024, 4096);
+          tc::mma_tf32_ss(tmem, ah, bh, idsc, (i > 0 || kg > 0) ? 1u : 0u);
+          tc::mma_tf32_ss(tmem, ah, bl, idsc, 1u);
+          tc::mma_tf32_ss(tmem, al, bh, idsc, 1u);
+        }
+        tc::mma_commit(empty + j);
+        if (i == nst - 1) tc::mma_commit(done);
+      }
+      __syncwarp();
+    }
+  } else {
+    const int t = threadIdx.x - 64;              // 0..127
+    for (int i = 0; i < nst; ++i) {
+      const int j = i % WG_NS;
+      tc::mbar_wait(full + j, (i / WG_NS) & 1);
+      uint8_t *st = stage(j);
+      const long r0 = rb + long(i) * 32;
+      // X raw -> X lo (boxes 0..nbx), Y raw -> Y lo; rows beyond this CTA's range -> 0
+      for (int f = t; f < 2 * 4 * 256; f += 128) {          // 2 operands x 4 boxes x 256 float4
+        const int op = f >> 10, b = (f >> 8) & 3, q4 = f & 255;
+        if (b >= (op == 0 ? nbx : nby)) continue;
+        float4 *raw = reinterpret_cast<float4 *>(st + op * 32768 + b * 4096) + q4;
+        float4 *lo = reinterpret_cast<float4 *>(st + op * 32768 + 16384 + b * 4096) + q4;
+        const int rr = q4 >> 3;                               // 8 float4 per 128-byte row
+        float4 v = *raw;
+        if (r0 + rr >= re) {
+          v = make_float4(0.f, 0.f, 0.f, 0.f);
+          *raw = v;
+        }
+        float4 l;
+        l.x = v.x - __uint_as_float(__float_as_uint(v.x) & 0xFFFFE000u);
+        l.y = v.y - __uint_as_float(__float_as_uint(v.y) & 0xFFFFE000u);
+        l.z = v.z - __uint_as_float(__float_as_uint(v.z) & 0xFFFFE000u);
+        l.w = v.w - __uint_as_float(__float_as_uint(v.w) & 0xFFFFE000u);
+        *lo = l;
+      }
+      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+      tc::mbar_arrive(lo_ready + j);
+    }
+    // epilogue: thread = output row a (TMEM lane), columns b
+    if (nst > 0) {
+      tc::mbar_wait(done, 0);
+      tc::fence_after_sync();
+    }
+    const int q = warp & 3, row = q * 32 + lane;
+    const uint32_t lane_base = tmem + (uint32_t(q * 32) << 16);
+    float *out = partial + long(blockIdx.x) * A * Bn + long(row) * Bn;
+    for (int c0 = 0; c0 < Npad; c0 += 16) {
+      uint32_t r[16];
+      if (nst > 0) {
+        tc::tmem_ld16(lane_base + c0, r);
+        tc::tmem_ld_wait();
+      } else {
+#pragma unroll
+        for (int u = 0; u < 16; ++u) r[u] = 0u;
+      }
+      if (row < A)
+#pragma unroll
+        for (int u = 0; u < 16; ++u)
+          if (c0 + u < Bn) out[c0 + u] = __uint_as_float(r[u]);
+    }
+  }
+  tc::fence_before_sync();
+  __syncthreads();
+  tc::fence_after_sync();
+  if (warp == 1) tc::tmem_dealloc<128>(tmem);
+}
+
 typedef CUresult (*PFN_encodeTiled)(CUtensorMap *, CUtensorMapDataType, cuuint32_t, void *,
                                     const cuuint64_t *, const cuuint64_t *, const cuuint32_t *,
                                     const cuuint32_t *, CUtensorMapInterleave, CUtensorMapSwizzle,
@@ -529,6 +671,44 @@ template <class Kern> void set_smem(Kern k, size_t bytes) {
     cudaError_t e_ = cudaGetLastError();            \
     if (e_ != cudaSuccess) return -int(e_);         \
   } while (0)
+
+static bool encode_rows_map32(CUtensorMap *m, const float *A, long R, int K) {
+  static PFN_encodeTiled fn = nullptr;
+  if (!fn) {
+    void *p = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) != cudaSuccess ||
+        q != cudaDriverEntryPointSuccess || !p)
+      return false;
+    fn = reinterpret_cast<PFN_encodeTiled>(p);
+  }
+  const cuuint64_t dims[2] = {cuuint64_t(K), cuuint64_t(R)};
+  const cuuint64_t strides[1] = {cuuint64_t(K) * 4};
+  const cuuint32_t box[2] = {32, 32};
+  const cuuint32_t estr[2] = {1, 1};
+  return fn(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, const_cast<float *>(A), dims, strides, box, estr,
+            CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+            CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
+bool wgrad_tc_supported(int A, int Bn) {
+  return A >= 32 && A <= 128 && A % 32 == 0 && Bn >= 16 && Bn <= 128 && Bn % 16 == 0;
+}
+
+// partial must hold splits * A * Bn floats; returns the number of launches (1) or -err.
+int launch_wgrad_tc(const occu_ctx *ctx, const float *X, int A, const float *Y, int Bn, long R,
+                    int splits, float *partial, cudaStream_t st) {
+  CUtensorMap xm, ym;
+  if (!encode_rows_map32(&xm, X, R, A) || !encode_rows_map32(&ym, Y, R, Bn))
+    return -int(cudaErrorInvalidValue);
+  const size_t smem = 1024 + WG_NS * 65536 + 256;
+  set_smem(wgrad_tc_kernel, smem);
+  OCCU_PROF_BEGIN(ctx, "wgrad_tc", st);
+  wgrad_tc_kernel<<<splits, WG_NTH, smem, st>>>(xm, ym, A, Bn, R, splits, partial);
+  OCCU_PROF_END(ctx);
+  TC_CHECK();
+  return 1;
+}
 
 bool tc_supported(const occu_config &c) {
   return (c.d == 64 || c.d == 128) && c.F_n <= 128;

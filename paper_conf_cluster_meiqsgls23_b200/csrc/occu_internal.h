@@ -118,6 +118,9 @@ struct FwdLayerArgs {
 int launch_forward_layer(const occu_ctx *ctx, const DevCsr &csr, const FwdLayerArgs &a,
                          cudaStream_t st);
 bool tc_supported(const occu_config &c);
+bool wgrad_tc_supported(int A, int Bn);
+int launch_wgrad_tc(const occu_ctx *ctx, const float *X, int A, const float *Y, int Bn, long R,
+                    int splits, float *partial, cudaStream_t st);
 size_t tc_partial_floats(int E, int D);
 int launch_forward_layer_tc(const occu_ctx *ctx, const DevCsr &csr, const FwdLayerArgs &a,
                             float *partial, cudaStream_t st);
