@@ -754,6 +754,41 @@ __global__ void __launch_bounds__(NT) wgrad_partial_kernel(const float *__restri
   }
 }
 
+// Skinny weight gradients (A*Bn <= 512, e.g. dW_e of layer 1 with F_e = 4, [da_s; da_d]):
+// thread o owns outputs o and o+256; rows staged through smem in chunks of 32.
+__global__ void __launch_bounds__(NT) wgrad_skinny_kernel(const float *__restrict__ X, int A,
+                                                          const float *__restrict__ Y, int Bn,
+                                                          long R, int splits,
+                                                          float *__restrict__ partial) {
+  __shared__ float Xs[WG_R][129];
+  __shared__ float Ys[WG_R][129];
+  const int n = A * Bn;
+  const long per = (R + splits - 1) / splits;
+  const long r0 = blockIdx.x * per, r1 = min(R, r0 + per);
+  float acc0 = 0.f, acc1 = 0.f;
+  const int o0 = threadIdx.x, o1 = threadIdx.x + NT;
+  const int a0 = o0 / Bn, b0 = o0 % Bn, a1 = o1 / Bn, b1 = o1 % Bn;
+  for (long rb = r0; rb < r1; rb += WG_R) {
+    __syncthreads();
+    for (int idx = threadIdx.x; idx < WG_R * A; idx += NT) {
+      const int rr = idx / A, cc = idx % A;
+      Xs[rr][cc] = rb + rr < r1 ? X[(rb + rr) * A + cc] : 0.f;
+    }
+    for (int idx = threadIdx.x; idx < WG_R * Bn; idx += NT) {
+      const int rr = idx / Bn, cc = idx % Bn;
+      Ys[rr][cc] = rb + rr < r1 ? Y[(rb + rr) * Bn + cc] : 0.f;
+    }
+    __syncthreads();
+    if (o0 < n)
+      for (int rr = 0; rr < WG_R; ++rr) acc0 = fmaf(Xs[rr][a0], Ys[rr][b0], acc0);
+    if (o1 < n)
+      for (int rr = 0; rr < WG_R; ++rr) acc1 = fmaf(Xs[rr][a1], Ys[rr][b1], acc1);
+  }
+  float *out = partial + long(blockIdx.x) * n;
+  if (o0 < n) out[o0] = acc0;
+  if (o1 < n) out[o1] = acc1;
+}
+
 __global__ void wgrad_reduce_kernel(const float *__restrict__ partial, int splits, long n,
                                     float *__restrict__ out) {
   for (long i = blockIdx.x * long(blockDim.x) + threadIdx.x; i < n; i += long(gridDim.x) * blockDim.x) {
@@ -918,6 +953,20 @@ static int wgrad(occu_ctx *ctx, const float *X, int A, const float *Y, int Bn, l
     LAUNCH_CHECK();
     return r + 1;
   }
+  if (n <= 2 * NT && A <= 128 && Bn <= 128) {
+    const int sp = 2 * ctx->num_sms;
+    if (ctx->ws.partial.ensure(size_t(sp) * n * 4) != cudaSuccess) return -int(cudaErrorMemoryAllocation);
+    float *part = ctx->ws.partial.as<float>();
+    OCCU_PROF_BEGIN(ctx, "wgrad_skinny", st);
+    wgrad_skinny_kernel<<<sp, NT, 0, st>>>(X, A, Y, Bn, R, sp, part);
+    OCCU_PROF_END(ctx);
+    LAUNCH_CHECK();
+    OCCU_PROF_BEGIN(ctx, "wgrad_reduce", st);
+    wgrad_reduce_kernel<<<grid_for(n, 256, 1024), 256, 0, st>>>(part, sp, n, out);
+    OCCU_PROF_END(ctx);
+    LAUNCH_CHECK();
+    return 2;
+  }
   if (ctx->ws.partial.ensure(size_t(splits) * n * 4) != cudaSuccess) return -int(cudaErrorMemoryAllocation);
   float *part = ctx->ws.partial.as<float>();
   OCCU_PROF_BEGIN(ctx, "wgrad_partial", st);
@@ -973,7 +1022,39 @@ static int backward_layer_impl(occu_ctx *ctx, const DevCsr &csr, const BwdLayerA
   const int sms = ctx->num_sms;
   int n = 0;
   float *de = w.deA.as<float>();
-  if (csr.E > 0) {
+  const bool tc = ctx->path == 0 && tc_supported(cf);
+  int r;
+  if (tc && csr.E > 0) {
+    // a10 on tensor cores: g recompute + softmax backward, W_mᵀ dv, z recompute + σ', W_eᵀ dz
+    if ((r = launch_bwd_gate_tc(ctx, csr, a.e, P + L.W_m[i], a.dh, a.h, a.hbar, w.MG.as<float>(),
+                                w.DV.as<float>(), st)) < 0) return r;
+    n += r;
+    if ((r = launch_plain_tc(ctx, w.DV.as<float>(), D, csr.E, P + L.W_m[i], 1, a.de_out, de,
+                             "de_tc", st)) < 0) return r;
+    n += r;
+    if (a.Ke > 16) {
+      if ((r = launch_bwd_edge_tc(ctx, csr, a.e_in, a.Ke, P + L.W_e[i], a.e, de, a.p, a.q,
+                                  w.DZ.as<float>(), w.dalpha.as<float>(), st)) < 0) return r;
+      n += r;
+    } else {
+      const int tiles = (csr.E + BM - 1) / BM;
+      const int KS = a.Ke > D ? a.Ke : D;
+      const size_t smB = (size_t(a.Ke) * D + BM * (KS + 4) + BM) * 4;
+      set_smem(edge_bwd_e_kernel<D>, smB);
+      OCCU_PROF_BEGIN(ctx, "edge_bwd_e", st);
+      edge_bwd_e_kernel<D><<<grid_for(tiles, 1, sms), NT, smB, st>>>(
+          a.e_in, a.Ke, a.e, de, P + L.W_e[i], a.p, a.q, csr.in_src, csr.in_dst, csr.E,
+          w.DZ.as<float>(), w.dalpha.as<float>(), nullptr);
+      OCCU_PROF_END(ctx);
+      LAUNCH_CHECK();
+      ++n;
+    }
+    if (a.de_prev) {
+      if ((r = launch_plain_tc(ctx, w.DZ.as<float>(), D, csr.E, P + L.W_e[i], 1, nullptr,
+                               a.de_prev, "de_prev_tc", st)) < 0) return r;
+      n += r;
+    }
+  } else if (csr.E > 0) {
     const size_t smA = (2 * D * D + BM * (D + 4)) * 4 + 2 * BM * 4;
     set_smem(edge_bwd_m_kernel<D>, smA);
     const int tiles = (csr.E + BM - 1) / BM;
@@ -1002,7 +1083,6 @@ static int backward_layer_impl(occu_ctx *ctx, const DevCsr &csr, const BwdLayerA
   OCCU_PROF_END(ctx);
   LAUNCH_CHECK();
   ++n;
-  int r;
   // dW_m = DVᵀ E' ; dW_e = DZᵀ E_in ; dW_u = dPᵀ H_in ; [da_s; da_d] = [dp dq]ᵀ h̄
   if ((r = wgrad(ctx, w.DV.as<float>(), D, a.e, D, csr.E, G + L.W_m[i], st)) < 0) return r;
   n += r;
@@ -1012,7 +1092,11 @@ static int backward_layer_impl(occu_ctx *ctx, const DevCsr &csr, const BwdLayerA
   n += r;
   if ((r = wgrad(ctx, w.dpq.as<float>(), 2, a.hbar, D, csr.N, G + L.a_s[i], st)) < 0) return r;
   n += r;
-  if (a.dh_prev && csr.N > 0) {   // dh^{i-1} = dP W_u  (K == D for i > 0)
+  if (a.dh_prev && csr.N > 0 && tc) {   // dh^{i-1} = dP W_u on tensor cores
+    if ((r = launch_plain_tc(ctx, w.dP.as<float>(), D, csr.N, P + L.W_u[i], 1, nullptr, a.dh_prev,
+                             "dh_prev_tc", st)) < 0) return r;
+    n += r;
+  } else if (a.dh_prev && csr.N > 0) {   // dh^{i-1} = dP W_u  (K == D for i > 0)
     const size_t sm1 = (size_t(D) * D + BM * (D + 4)) * 4;
     set_smem(node_gemm_kernel<D, 1>, sm1);
     const int tiles = (csr.N + BM - 1) / BM;

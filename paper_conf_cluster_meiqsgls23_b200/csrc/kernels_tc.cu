@@ -44,6 +44,10 @@ constexpr int TM = 128;
 constexpr int NTH = 704;          // warp 0 producer, 1 MMA, 2-5 converters, 6-21 epilogue
 constexpr uint32_t TMEM_COLS = 512;
 constexpr int EPI_NODE = 0, EPI_EDGE = 1, EPI_GATE = 2;
+// backward epilogues (SURVEY §8(c) step BW)
+constexpr int EPI_PLAIN = 3;      // out = acc (+ add)
+constexpr int EPI_GATEBWD = 4;    // g = softmax(acc); dm = dA[t]; MG = dm ⊙ g; DV = g ⊙ (dm ⊙ h̄[s] - <g, dm ⊙ h̄[s]>)
+constexpr int EPI_EDGEBWD = 5;    // z = acc; dy = de ⊙ e' ⊙ σ(-αz); dα = <dy, z>; DZ = α dy
 
 
 
@@ -69,6 +73,13 @@ struct RowGemmArgs {
   const float *pin, *qin;  // EDGE: p, q of the layer
   const int32_t *src, *dst;
   float slope;
+  int transW;              // W given as [K][D] (the row-GEMM uses its transpose)
+  const float *add;        // PLAIN: [R][D] addend (nullable)
+  float *out2;             // GATEBWD: DV
+  const float *dh, *h, *hbar, *e, *de;
+  const int32_t *in_ptr;
+  int mean;
+  float *dal;              // EDGEBWD: dα [R]
 };
 
 struct Smem {
@@ -189,7 +200,7 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
 
   // ---- weight scale 2^f (block max |W|) and fp16x2 SW128 images ------------
   float wmx = 0.f;
-  for (int i = threadIdx.x; i < D * K; i += NTH) wmx = fmaxf(wmx, fabsf(__ldg(a.W + i)));
+  for (int i = threadIdx.x; i < D * K; i += NTH) wmx = fmaxf(wmx, fabsf(__ldg(a.W + i)));   // any layout
 #pragma unroll
   for (int o = 16; o > 0; o >>= 1) wmx = fmaxf(wmx, __shfl_xor_sync(0xffffffffu, wmx, o));
   if (lane == 0) s.red[warp] = wmx;
@@ -204,8 +215,10 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
   const float wscale = ldexpf(1.f, fexp);
   for (int i = threadIdx.x; i < D * (Kpad / 2); i += NTH) {
     const int n = i / (Kpad / 2), k = 2 * (i % (Kpad / 2));
-    const float v0 = k < K ? __ldg(a.W + long(n) * K + k) * wscale : 0.f;
-    const float v1 = k + 1 < K ? __ldg(a.W + long(n) * K + k + 1) * wscale : 0.f;
+    const long i0 = a.transW ? long(k) * D + n : long(n) * K + k;
+    const long i1 = a.transW ? long(k + 1) * D + n : long(n) * K + k + 1;
+    const float v0 = k < K ? __ldg(a.W + i0) * wscale : 0.f;
+    const float v1 = k + 1 < K ? __ldg(a.W + i1) * wscale : 0.f;
     uint32_t hi, lo;
     split2(v0, v1, hi, lo);
     const uint32_t off = tc::sw128_offset_f16(n, k, D);
@@ -340,13 +353,13 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
       const int nrows = min(TM, int(a.R - r0));
       const bool live = row < nrows;
       float aux = 0.f;
-      if (EPI == EPI_EDGE && hf == 0 && live)
+      if ((EPI == EPI_EDGE || EPI == EPI_EDGEBWD) && hf == 0 && live)
         aux = __ldg(a.pin + __ldg(a.src + r0 + row)) + __ldg(a.qin + __ldg(a.dst + r0 + row));  // α (R1)
       tc::mbar_wait(s.eready + (i & 3), (i >> 2) & 1);
       const int er = s.erow[(i & 3) * 128 + row];
       tc::mbar_wait(s.accfull + j, (i >> 1) & 1);
       tc::fence_after_sync();
-      if (EPI == EPI_EDGE) {
+      if (EPI == EPI_EDGE || EPI == EPI_EDGEBWD) {
         if (hf == 0) xg[row] = aux;
         group_bar(g);
         aux = xg[row];
@@ -356,7 +369,136 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
       const long wrow0 = r0 + qd * 32;
       const int wrows = max(0, min(32, nrows - qd * 32));
       const uint32_t acc = lane_base + acc_col(j) + cb;
-      if (EPI == EPI_GATE) {
+      if (EPI == EPI_PLAIN) {
+#pragma unroll 1
+        for (int c0 = 0; c0 < DH; c0 += 16) {
+          uint32_t r[16];
+          tc::tmem_ld16(acc + c0, r);
+          tc::tmem_ld_wait();
+          float o[16];
+#pragma unroll
+          for (int u = 0; u < 16; ++u) o[u] = __uint_as_float(r[u]) * un;
+          if (a.add && live) {
+            const float *ar = a.add + grow * D + cb + c0;
+#pragma unroll
+            for (int u = 0; u < 16; u += 4) {
+              const float4 x = __ldg(reinterpret_cast<const float4 *>(ar + u));
+              o[u] += x.x; o[u + 1] += x.y; o[u + 2] += x.z; o[u + 3] += x.w;
+            }
+          }
+          warp_store_chunk<D>(wbuf, a.out, wrow0, wrows, cb + c0, o, lane);
+        }
+      } else if (EPI == EPI_EDGEBWD) {
+        float dpart = 0.f;
+#pragma unroll 1
+        for (int c0 = 0; c0 < DH; c0 += 16) {
+          uint32_t r[16];
+          tc::tmem_ld16(acc + c0, r);
+          tc::tmem_ld_wait();
+          float o[16];
+          const float *er = a.e + grow * D + cb + c0, *dr = a.de + grow * D + cb + c0;
+#pragma unroll
+          for (int u = 0; u < 16; u += 4) {
+            float4 ev = make_float4(0.f, 0.f, 0.f, 0.f), dv = ev;
+            if (live) {
+              ev = __ldg(reinterpret_cast<const float4 *>(er + u));
+              dv = __ldg(reinterpret_cast<const float4 *>(dr + u));
+            }
+            const float evv[4] = {ev.x, ev.y, ev.z, ev.w}, dvv[4] = {dv.x, dv.y, dv.z, dv.w};
+#pragma unroll
+            for (int t = 0; t < 4; ++t) {
+              const float z = __uint_as_float(r[u + t]) * un;
+              // σ'(y) = σ(y)·σ(-y), y = α z (recomputed): no 1 - e' cancellation
+              const float dy = dvv[t] * evv[t] * fast_rcp(1.f + fast_exp(aux * z));
+              dpart = fmaf(dy, z, dpart);
+              o[u + t] = aux * dy;
+            }
+          }
+          warp_store_chunk<D>(wbuf, a.out, wrow0, wrows, cb + c0, o, lane);
+        }
+        xg[256 + hf * 128 + row] = dpart;
+        group_bar(g);
+        if (hf == 0 && live) a.dal[grow] = dpart + xg[256 + 128 + row];
+      } else if (EPI == EPI_GATEBWD) {
+        // softmax statistics (as the forward gate)
+        float m = -INFINITY;
+#pragma unroll
+        for (int c0 = 0; c0 < DH; c0 += 16) {
+          uint32_t r[16];
+          tc::tmem_ld16(acc + c0, r);
+          tc::tmem_ld_wait();
+#pragma unroll
+          for (int u = 0; u < 16; ++u) m = fmaxf(m, __uint_as_float(r[u]) * un);
+        }
+        xg[hf * 128 + row] = m;
+        group_bar(g);
+        m = fmaxf(m, xg[(hf ^ 1) * 128 + row]);
+        float sum = 0.f;
+#pragma unroll
+        for (int c0 = 0; c0 < DH; c0 += 16) {
+          uint32_t r[16];
+          tc::tmem_ld16(acc + c0, r);
+          tc::tmem_ld_wait();
+#pragma unroll
+          for (int u = 0; u < 16; ++u) sum += fast_exp(__uint_as_float(r[u]) * un - m);
+        }
+        xg[256 + hf * 128 + row] = sum;
+        group_bar(g);
+        sum = hf == 0 ? sum + xg[256 + 128 + row] : xg[256 + row] + sum;
+        const float inv = fast_rcp(sum);
+        // dA[t] = dh[t] ⊙ LReLU'(h[t]) (÷ deg for MEAN); gathers by destination / source
+        const int tn = live ? __ldg(a.dst + grow) : 0;
+        const int sn = live ? __ldg(a.src + grow) : 0;
+        float dscale = 1.f;
+        if (a.mean && live) {
+          const int deg = __ldg(a.in_ptr + tn + 1) - __ldg(a.in_ptr + tn);
+          dscale = float(deg > 0 ? deg : 1);
+        }
+        const float *dhr = a.dh + long(tn) * D + cb, *hr = a.h + long(tn) * D + cb;
+        const float *hbr = a.hbar + long(sn) * D + cb;
+        float dot = 0.f;
+        group_bar(g);          // everyone has read the (m, sum) exchange slots
+#pragma unroll 1
+        for (int pass = 0; pass < 2; ++pass) {
+#pragma unroll 1
+          for (int c0 = 0; c0 < DH; c0 += 16) {
+            uint32_t r[16];
+            tc::tmem_ld16(acc + c0, r);
+            tc::tmem_ld_wait();
+            float o[16];
+#pragma unroll
+            for (int u = 0; u < 16; u += 4) {
+              float4 d4 = make_float4(0.f, 0.f, 0.f, 0.f), h4 = d4, b4 = d4;
+              if (live) {
+                d4 = __ldg(reinterpret_cast<const float4 *>(dhr + c0 + u));
+                h4 = __ldg(reinterpret_cast<const float4 *>(hr + c0 + u));
+                b4 = __ldg(reinterpret_cast<const float4 *>(hbr + c0 + u));
+              }
+              const float dv[4] = {d4.x, d4.y, d4.z, d4.w}, hv[4] = {h4.x, h4.y, h4.z, h4.w};
+              const float bv[4] = {b4.x, b4.y, b4.z, b4.w};
+#pragma unroll
+              for (int t = 0; t < 4; ++t) {
+                const float gg = fast_exp(__uint_as_float(r[u + t]) * un - m) * inv;
+                float dm = dv[t] * (hv[t] > 0.f ? 1.f : a.slope);
+                if (a.mean) dm = dm / dscale;
+                const float dg = dm * bv[t];
+                if (pass == 0) {
+                  dot = fmaf(gg, dg, dot);
+                  o[u + t] = dm * gg;                              // MG
+                } else {
+                  o[u + t] = gg * (dg - dot);                      // DV
+                }
+              }
+            }
+            warp_store_chunk<D>(wbuf, pass == 0 ? a.out : a.out2, wrow0, wrows, cb + c0, o, lane);
+          }
+          if (pass == 0) {
+            xg[hf * 128 + row] = dot;
+            group_bar(g);
+            dot = hf == 0 ? dot + xg[128 + row] : xg[row] + dot;   // fixed order
+          }
+        }
+      } else if (EPI == EPI_GATE) {
         float m = -INFINITY;
 #pragma unroll
         for (int c0 = 0; c0 < DH; c0 += 16) {
@@ -777,6 +919,58 @@ static int tc_forward_layer_impl(const occu_ctx *ctx, const DevCsr &csr, const F
   // a5 + a6: gather + segmented sum (CUDA cores, warp per destination)
   if ((r = launch_gather_segsum(ctx, csr, a.g, a.hbar, a.h_out, st)) < 0) return r;
   return n + r;
+}
+
+// ---- backward row-GEMMs on tensor cores ------------------------------------
+template <int D>
+static int bwd_gate_impl(const occu_ctx *ctx, const DevCsr &csr, const float *e, const float *W_m,
+                         const float *dh, const float *h, const float *hbar, float *MG, float *DV,
+                         cudaStream_t st) {
+  RowGemmArgs r{};
+  r.slope = ctx->cfg.slope;
+  r.A = e; r.K = D; r.R = csr.E; r.W = W_m; r.out = MG; r.out2 = DV;
+  r.dh = dh; r.h = h; r.hbar = hbar; r.src = csr.in_src; r.dst = csr.in_dst;
+  r.in_ptr = csr.in_ptr; r.mean = ctx->cfg.aggr == OCCU_AGGR_MEAN;
+  return launch_rowgemm<D, EPI_GATEBWD>(ctx, r, "gate_bwd_tc", st);
+}
+template <int D>
+static int plain_impl(const occu_ctx *ctx, const float *A, int K, int R, const float *W, int transW,
+                      const float *add, float *out, const char *name, cudaStream_t st) {
+  RowGemmArgs r{};
+  r.slope = ctx->cfg.slope;
+  r.A = A; r.K = K; r.R = R; r.W = W; r.transW = transW; r.add = add; r.out = out;
+  return launch_rowgemm<D, EPI_PLAIN>(ctx, r, name, st);
+}
+template <int D>
+static int bwd_edge_impl(const occu_ctx *ctx, const DevCsr &csr, const float *e_in, int Ke,
+                         const float *W_e, const float *e, const float *de, const float *p,
+                         const float *q, float *DZ, float *dal, cudaStream_t st) {
+  RowGemmArgs r{};
+  r.slope = ctx->cfg.slope;
+  r.A = e_in; r.K = Ke; r.R = csr.E; r.W = W_e; r.out = DZ; r.dal = dal;
+  r.e = e; r.de = de; r.pin = p; r.qin = q; r.src = csr.in_src; r.dst = csr.in_dst;
+  return launch_rowgemm<D, EPI_EDGEBWD>(ctx, r, "edge_bwd_tc", st);
+}
+
+int launch_bwd_gate_tc(const occu_ctx *ctx, const DevCsr &csr, const float *e, const float *W_m,
+                       const float *dh, const float *h, const float *hbar, float *MG, float *DV,
+                       cudaStream_t st) {
+  if (csr.E <= 0) return 0;
+  return ctx->cfg.d == 64 ? bwd_gate_impl<64>(ctx, csr, e, W_m, dh, h, hbar, MG, DV, st)
+                          : bwd_gate_impl<128>(ctx, csr, e, W_m, dh, h, hbar, MG, DV, st);
+}
+int launch_plain_tc(const occu_ctx *ctx, const float *A, int K, int R, const float *W, int transW,
+                    const float *add, float *out, const char *name, cudaStream_t st) {
+  if (R <= 0) return 0;
+  return ctx->cfg.d == 64 ? plain_impl<64>(ctx, A, K, R, W, transW, add, out, name, st)
+                          : plain_impl<128>(ctx, A, K, R, W, transW, add, out, name, st);
+}
+int launch_bwd_edge_tc(const occu_ctx *ctx, const DevCsr &csr, const float *e_in, int Ke,
+                       const float *W_e, const float *e, const float *de, const float *p,
+                       const float *q, float *DZ, float *dal, cudaStream_t st) {
+  if (csr.E <= 0) return 0;
+  return ctx->cfg.d == 64 ? bwd_edge_impl<64>(ctx, csr, e_in, Ke, W_e, e, de, p, q, DZ, dal, st)
+                          : bwd_edge_impl<128>(ctx, csr, e_in, Ke, W_e, e, de, p, q, DZ, dal, st);
 }
 
 int launch_forward_layer_tc(const occu_ctx *ctx, const DevCsr &csr, const FwdLayerArgs &a,

@@ -119,6 +119,14 @@ int launch_forward_layer(const occu_ctx *ctx, const DevCsr &csr, const FwdLayerA
                          cudaStream_t st);
 bool tc_supported(const occu_config &c);
 bool wgrad_tc_supported(int A, int Bn);
+int launch_bwd_gate_tc(const occu_ctx *ctx, const DevCsr &csr, const float *e, const float *W_m,
+                       const float *dh, const float *h, const float *hbar, float *MG, float *DV,
+                       cudaStream_t st);
+int launch_plain_tc(const occu_ctx *ctx, const float *A, int K, int R, const float *W, int transW,
+                    const float *add, float *out, const char *name, cudaStream_t st);
+int launch_bwd_edge_tc(const occu_ctx *ctx, const DevCsr &csr, const float *e_in, int Ke,
+                       const float *W_e, const float *e, const float *de, const float *p,
+                       const float *q, float *DZ, float *dal, cudaStream_t st);
 int launch_wgrad_tc(const occu_ctx *ctx, const float *X, int A, const float *Y, int Bn, long R,
                     int splits, float *partial, cudaStream_t st);
 size_t tc_partial_floats(int E, int D);
