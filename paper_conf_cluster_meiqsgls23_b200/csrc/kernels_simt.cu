@@ -463,15 +463,25 @@ __global__ void head_bwd_reduce_kernel(const float *__restrict__ dy, const float
 }
 
 // dh^L_u = dr_{graph(u)} / n_{graph(u)}
+// h_mask != null: emit dA = dh ⊙ LReLU'(A) (÷ deg for MEAN; sign(A) = sign(h)) instead of dh.
 __global__ void broadcast_dh_kernel(const float *__restrict__ dr, const int32_t *__restrict__ node_graph,
                                     const int32_t *__restrict__ node_off, int N, int D,
-                                    float *__restrict__ dh) {
+                                    const float *__restrict__ h_mask, const int32_t *__restrict__ in_ptr,
+                                    int mean, float slope, float *__restrict__ dh) {
   const long total = long(N) * D;
   for (long i = blockIdx.x * long(blockDim.x) + threadIdx.x; i < total;
        i += long(gridDim.x) * blockDim.x) {
     const int u = int(i / D), k = int(i % D);
     const int b = node_graph[u];
-    dh[i] = dr[long(b) * D + k] / float(node_off[b + 1] - node_off[b]);
+    float v = dr[long(b) * D + k] / float(node_off[b + 1] - node_off[b]);
+    if (h_mask) {
+      v = v * lrelu_grad_from_out(h_mask[i], slope);
+      if (mean) {
+        const int deg = in_ptr[u + 1] - in_ptr[u];
+        v = v / float(deg > 0 ? deg : 1);
+      }
+    }
+    dh[i] = v;
   }
 }
 
@@ -666,10 +676,15 @@ __global__ void __launch_bounds__(NT) node_bwd_kernel(
     const float *__restrict__ hbar, const float *__restrict__ a_s, const float *__restrict__ a_d,
     const int32_t *__restrict__ out_ptr, const int32_t *__restrict__ out_pos,
     const int32_t *__restrict__ in_ptr, int N, float slope, float *__restrict__ dP,
-    float *__restrict__ dpq) {
+    float *__restrict__ dpq, float *__restrict__ da_part) {
+  // da_part != null: also accumulate [da_s; da_d] = Σ_u [dp_u; dq_u] h̄_u per warp (fixed
+  // node assignment) into da_part[warp][2][D] for a fixed-order reduction.
   constexpr int V = D / 32;
   const int lane = threadIdx.x & 31;
   const int warps = (gridDim.x * NT) / 32;
+  float das[V], dad[V];
+#pragma unroll
+  for (int c = 0; c < V; ++c) das[c] = dad[c] = 0.f;
   for (int u = (blockIdx.x * NT + threadIdx.x) / 32; u < N; u += warps) {
     float acc[V];
 #pragma unroll
@@ -690,10 +705,20 @@ __global__ void __launch_bounds__(NT) node_bwd_kernel(
       const float v = acc[c] + dp * a_s[ch] + dq * a_d[ch];
       const float hb = hbar[long(u) * D + ch];
       dP[long(u) * D + ch] = v * lrelu_grad_from_out(hb, slope);
+      das[c] = fmaf(dp, hb, das[c]);
+      dad[c] = fmaf(dq, hb, dad[c]);
     }
     if (lane == 0) {
       dpq[2 * long(u)] = dp;
       dpq[2 * long(u) + 1] = dq;
+    }
+  }
+  if (da_part) {
+    const long wg = (blockIdx.x * NT + threadIdx.x) / 32;
+#pragma unroll
+    for (int c = 0; c < V; ++c) {
+      da_part[wg * 2 * D + lane * V + c] = das[c];
+      da_part[wg * 2 * D + D + lane * V + c] = dad[c];
     }
   }
 }
@@ -1003,8 +1028,11 @@ int launch_head_backward(occu_ctx *ctx, const DevCsr &csr, const float *targets,
   OCCU_PROF_END(ctx);
   LAUNCH_CHECK();
   OCCU_PROF_BEGIN(ctx, "broadcast_dh", st);
+  const bool tcb = ctx->path == 0 && tc_supported(cf);    // TC backward consumes dA directly
   broadcast_dh_kernel<<<grid_for(long(csr.N) * cf.d, 256, 8192), 256, 0, st>>>(
-      w.dr.as<float>(), csr.node_graph, csr.node_off, csr.N, cf.d, w.dh.as<float>());
+      w.dr.as<float>(), csr.node_graph, csr.node_off, csr.N, cf.d,
+      tcb ? w.h[cf.L - 1].as<float>() : nullptr, csr.in_ptr, cf.aggr == OCCU_AGGR_MEAN, cf.slope,
+      w.dh.as<float>());
   OCCU_PROF_END(ctx);
   LAUNCH_CHECK();
   return 3;
@@ -1026,7 +1054,7 @@ static int backward_layer_impl(occu_ctx *ctx, const DevCsr &csr, const BwdLayerA
   int r;
   if (tc && csr.E > 0) {
     // a10 on tensor cores: g recompute + softmax backward, W_mᵀ dv, z recompute + σ', W_eᵀ dz
-    if ((r = launch_bwd_gate_tc(ctx, csr, a.e, P + L.W_m[i], a.dh, a.h, a.hbar, w.MG.as<float>(),
+    if ((r = launch_bwd_gate_tc(ctx, csr, a.e, P + L.W_m[i], a.dh, nullptr, a.hbar, w.MG.as<float>(),
                                 w.DV.as<float>(), st)) < 0) return r;
     n += r;
     if ((r = launch_plain_tc(ctx, w.DV.as<float>(), D, csr.E, P + L.W_m[i], 1, a.de_out, de,
@@ -1076,13 +1104,28 @@ static int backward_layer_impl(occu_ctx *ctx, const DevCsr &csr, const BwdLayerA
     LAUNCH_CHECK();
     ++n;
   }
+  const int nb_blocks = tc ? 2 * sms : grid_for(long(csr.N) * 32, NT, 16 * sms);
+  const int nb_warps = nb_blocks * (NT / 32);
+  float *da_part = nullptr;
+  if (tc) {
+    if (w.dpart.ensure(size_t(nb_warps) * 2 * D * 4) != cudaSuccess) return -int(cudaErrorMemoryAllocation);
+    da_part = w.dpart.as<float>();
+  }
   OCCU_PROF_BEGIN(ctx, "node_bwd", st);
-  node_bwd_kernel<D><<<grid_for(long(csr.N) * 32, NT, 16 * sms), NT, 0, st>>>(
+  node_bwd_kernel<D><<<nb_blocks, NT, 0, st>>>(
       w.MG.as<float>(), w.dalpha.as<float>(), a.hbar, P + L.a_s[i], P + L.a_d[i], csr.out_ptr,
-      csr.out_pos, csr.in_ptr, csr.N, cf.slope, w.dP.as<float>(), w.dpq.as<float>());
+      csr.out_pos, csr.in_ptr, csr.N, cf.slope, w.dP.as<float>(), w.dpq.as<float>(), da_part);
   OCCU_PROF_END(ctx);
   LAUNCH_CHECK();
   ++n;
+  if (tc) {
+    OCCU_PROF_BEGIN(ctx, "wgrad_reduce", st);
+    wgrad_reduce_kernel<<<grid_for(2 * D, 256, 1024), 256, 0, st>>>(da_part, nb_warps, 2 * D,
+                                                                     G + L.a_s[i]);
+    OCCU_PROF_END(ctx);
+    LAUNCH_CHECK();
+    ++n;
+  }
   // dW_m = DVᵀ E' ; dW_e = DZᵀ E_in ; dW_u = dPᵀ H_in ; [da_s; da_d] = [dp dq]ᵀ h̄
   if ((r = wgrad(ctx, w.DV.as<float>(), D, a.e, D, csr.E, G + L.W_m[i], st)) < 0) return r;
   n += r;
@@ -1090,11 +1133,13 @@ static int backward_layer_impl(occu_ctx *ctx, const DevCsr &csr, const BwdLayerA
   n += r;
   if ((r = wgrad(ctx, w.dP.as<float>(), D, a.h_in, a.K, csr.N, G + L.W_u[i], st)) < 0) return r;
   n += r;
-  if ((r = wgrad(ctx, w.dpq.as<float>(), 2, a.hbar, D, csr.N, G + L.a_s[i], st)) < 0) return r;
-  n += r;
+  if (!tc) {
+    if ((r = wgrad(ctx, w.dpq.as<float>(), 2, a.hbar, D, csr.N, G + L.a_s[i], st)) < 0) return r;
+    n += r;
+  }
   if (a.dh_prev && csr.N > 0 && tc) {   // dh^{i-1} = dP W_u on tensor cores
     if ((r = launch_plain_tc(ctx, w.dP.as<float>(), D, csr.N, P + L.W_u[i], 1, nullptr, a.dh_prev,
-                             "dh_prev_tc", st)) < 0) return r;
+                             "dh_prev_tc", st, a.h_in, csr.in_ptr)) < 0) return r;
     n += r;
   } else if (a.dh_prev && csr.N > 0) {   // dh^{i-1} = dP W_u  (K == D for i > 0)
     const size_t sm1 = (size_t(D) * D + BM * (D + 4)) * 4;

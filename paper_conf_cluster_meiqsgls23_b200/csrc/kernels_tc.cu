@@ -77,6 +77,7 @@ struct RowGemmArgs {
   const float *add;        // PLAIN: [R][D] addend (nullable)
   float *out2;             // GATEBWD: DV
   const float *dh, *h, *hbar, *e, *de;
+  const float *mask_h;     // PLAIN: multiply row by LReLU'(mask_h row) (÷ deg for MEAN) -> dA
   const int32_t *in_ptr;
   int mean;
   float *dal;              // EDGEBWD: dα [R]
@@ -378,6 +379,24 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
           float o[16];
 #pragma unroll
           for (int u = 0; u < 16; ++u) o[u] = __uint_as_float(r[u]) * un;
+          if (a.mask_h && live) {
+            const float *mr = a.mask_h + grow * D + cb + c0;
+            float dsc = 1.f;
+            if (a.mean) {
+              const int deg = __ldg(a.in_ptr + grow + 1) - __ldg(a.in_ptr + grow);
+              dsc = float(deg > 0 ? deg : 1);
+            }
+#pragma unroll
+            for (int u = 0; u < 16; u += 4) {
+              const float4 x = __ldg(reinterpret_cast<const float4 *>(mr + u));
+              const float xv[4] = {x.x, x.y, x.z, x.w};
+#pragma unroll
+              for (int t = 0; t < 4; ++t) {
+                o[u + t] *= xv[t] > 0.f ? 1.f : a.slope;
+                if (a.mean) o[u + t] = o[u + t] / dsc;
+              }
+            }
+          }
           if (a.add && live) {
             const float *ar = a.add + grow * D + cb + c0;
 #pragma unroll
@@ -450,11 +469,12 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
         const int tn = live ? __ldg(a.dst + grow) : 0;
         const int sn = live ? __ldg(a.src + grow) : 0;
         float dscale = 1.f;
-        if (a.mean && live) {
+        const bool is_dA = a.h == nullptr;
+        if (!is_dA && a.mean && live) {
           const int deg = __ldg(a.in_ptr + tn + 1) - __ldg(a.in_ptr + tn);
           dscale = float(deg > 0 ? deg : 1);
         }
-        const float *dhr = a.dh + long(tn) * D + cb, *hr = a.h + long(tn) * D + cb;
+        const float *dhr = a.dh + long(tn) * D + cb, *hr = is_dA ? dhr : a.h + long(tn) * D + cb;
         const float *hbr = a.hbar + long(sn) * D + cb;
         float dot = 0.f;
         group_bar(g);          // everyone has read the (m, sum) exchange slots
@@ -471,7 +491,7 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
               float4 d4 = make_float4(0.f, 0.f, 0.f, 0.f), h4 = d4, b4 = d4;
               if (live) {
                 d4 = __ldg(reinterpret_cast<const float4 *>(dhr + c0 + u));
-                h4 = __ldg(reinterpret_cast<const float4 *>(hr + c0 + u));
+                if (!is_dA) h4 = __ldg(reinterpret_cast<const float4 *>(hr + c0 + u));
                 b4 = __ldg(reinterpret_cast<const float4 *>(hbr + c0 + u));
               }
               const float dv[4] = {d4.x, d4.y, d4.z, d4.w}, hv[4] = {h4.x, h4.y, h4.z, h4.w};
@@ -479,8 +499,11 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
 #pragma unroll
               for (int t = 0; t < 4; ++t) {
                 const float gg = fast_exp(__uint_as_float(r[u + t]) * un - m) * inv;
-                float dm = dv[t] * (hv[t] > 0.f ? 1.f : a.slope);
-                if (a.mean) dm = dm / dscale;
+                float dm = dv[t];
+                if (!is_dA) {
+                  dm = dm * (hv[t] > 0.f ? 1.f : a.slope);
+                  if (a.mean) dm = dm / dscale;
+                }
                 const float dg = dm * bv[t];
                 if (pass == 0) {
                   dot = fmaf(gg, dg, dot);
@@ -935,10 +958,12 @@ static int bwd_gate_impl(const occu_ctx *ctx, const DevCsr &csr, const float *e,
 }
 template <int D>
 static int plain_impl(const occu_ctx *ctx, const float *A, int K, int R, const float *W, int transW,
-                      const float *add, float *out, const char *name, cudaStream_t st) {
+                      const float *add, float *out, const char *name, cudaStream_t st,
+                      const float *mask_h, const int32_t *in_ptr) {
   RowGemmArgs r{};
   r.slope = ctx->cfg.slope;
   r.A = A; r.K = K; r.R = R; r.W = W; r.transW = transW; r.add = add; r.out = out;
+  r.mask_h = mask_h; r.in_ptr = in_ptr; r.mean = ctx->cfg.aggr == OCCU_AGGR_MEAN;
   return launch_rowgemm<D, EPI_PLAIN>(ctx, r, name, st);
 }
 template <int D>
@@ -960,10 +985,11 @@ int launch_bwd_gate_tc(const occu_ctx *ctx, const DevCsr &csr, const float *e, c
                           : bwd_gate_impl<128>(ctx, csr, e, W_m, dh, h, hbar, MG, DV, st);
 }
 int launch_plain_tc(const occu_ctx *ctx, const float *A, int K, int R, const float *W, int transW,
-                    const float *add, float *out, const char *name, cudaStream_t st) {
+                    const float *add, float *out, const char *name, cudaStream_t st,
+                    const float *mask_h, const int32_t *in_ptr) {
   if (R <= 0) return 0;
-  return ctx->cfg.d == 64 ? plain_impl<64>(ctx, A, K, R, W, transW, add, out, name, st)
-                          : plain_impl<128>(ctx, A, K, R, W, transW, add, out, name, st);
+  return ctx->cfg.d == 64 ? plain_impl<64>(ctx, A, K, R, W, transW, add, out, name, st, mask_h, in_ptr)
+                          : plain_impl<128>(ctx, A, K, R, W, transW, add, out, name, st, mask_h, in_ptr);
 }
 int launch_bwd_edge_tc(const occu_ctx *ctx, const DevCsr &csr, const float *e_in, int Ke,
                        const float *W_e, const float *e, const float *de, const float *p,

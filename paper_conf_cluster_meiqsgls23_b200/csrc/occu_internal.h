@@ -47,6 +47,7 @@ struct Workspace {
   // backward scratch
   DevBuf dy, dc, dr, dh, dhprev, dP, MG, DV, DZ, deA, deB, dalpha, dpq, partial, loss;
   DevBuf tcpart;           // tensor-core aggregation: boundary-segment partials
+  DevBuf dpart;            // per-warp [da_s; da_d] partials
   void release_all();
 };
 
@@ -123,7 +124,8 @@ int launch_bwd_gate_tc(const occu_ctx *ctx, const DevCsr &csr, const float *e, c
                        const float *dh, const float *h, const float *hbar, float *MG, float *DV,
                        cudaStream_t st);
 int launch_plain_tc(const occu_ctx *ctx, const float *A, int K, int R, const float *W, int transW,
-                    const float *add, float *out, const char *name, cudaStream_t st);
+                    const float *add, float *out, const char *name, cudaStream_t st,
+                    const float *mask_h = nullptr, const int32_t *in_ptr = nullptr);
 int launch_bwd_edge_tc(const occu_ctx *ctx, const DevCsr &csr, const float *e_in, int Ke,
                        const float *W_e, const float *e, const float *de, const float *p,
                        const float *q, float *DZ, float *dal, cudaStream_t st);

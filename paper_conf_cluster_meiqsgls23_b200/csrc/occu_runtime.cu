@@ -44,7 +44,7 @@ void DevBuf::release() {
 void Workspace::release_all() {
   DevBuf *bufs[] = {&node_feat, &edge_feat, &targets, &out_occ, &csr, &e0, &g, &r, &c, &yhat,
                     &dy, &dc, &dr, &dh, &dhprev, &dP, &MG, &DV, &DZ, &deA, &deB, &dalpha,
-                    &dpq, &partial, &loss, &tcpart};
+                    &dpq, &partial, &loss, &tcpart, &dpart};
   for (DevBuf *b : bufs) b->release();
   for (auto *v : {&hbar, &p, &q, &e, &h})
     for (DevBuf &b : *v) b.release();
