@@ -713,12 +713,19 @@ __global__ void __launch_bounds__(NT) node_bwd_kernel(
       dpq[2 * long(u) + 1] = dq;
     }
   }
-  if (da_part) {
-    const long wg = (blockIdx.x * NT + threadIdx.x) / 32;
+  if (da_part) {   // per-block partial: warps combined in fixed warp order through smem
+    __shared__ float red[NT / 32][2 * D];
+    const int wl = threadIdx.x / 32;
 #pragma unroll
     for (int c = 0; c < V; ++c) {
-      da_part[wg * 2 * D + lane * V + c] = das[c];
-      da_part[wg * 2 * D + D + lane * V + c] = dad[c];
+      red[wl][lane * V + c] = das[c];
+      red[wl][D + lane * V + c] = dad[c];
+    }
+    __syncthreads();
+    for (int o = threadIdx.x; o < 2 * D; o += NT) {
+      float acc2 = 0.f;
+      for (int w2 = 0; w2 < NT / 32; ++w2) acc2 += red[w2][o];
+      da_part[long(blockIdx.x) * 2 * D + o] = acc2;
     }
   }
 }
@@ -812,6 +819,29 @@ __global__ void __launch_bounds__(NT) wgrad_skinny_kernel(const float *__restric
   float *out = partial + long(blockIdx.x) * n;
   if (o0 < n) out[o0] = acc0;
   if (o1 < n) out[o1] = acc1;
+}
+
+// out[o] = Σ_k partial[k][o] with the split range cut into LANES interleaved
+// sub-sums (lane l takes k ≡ l mod LANES) combined in lane order: fixed order,
+// LANES-way parallel per output.
+template <int LANES>
+__global__ void __launch_bounds__(256) split_reduce_kernel(const float *__restrict__ partial,
+                                                           int splits, long n,
+                                                           float *__restrict__ out) {
+  constexpr int OPB = 256 / LANES;            // outputs per block
+  __shared__ float red[LANES][OPB];
+  const int ol = threadIdx.x % OPB, l = threadIdx.x / OPB;
+  const long o = long(blockIdx.x) * OPB + ol;
+  float acc = 0.f;
+  if (o < n)
+    for (int k = l; k < splits; k += LANES) acc += partial[long(k) * n + o];
+  red[l][ol] = acc;
+  __syncthreads();
+  if (l == 0 && o < n) {
+    float t = 0.f;
+    for (int j = 0; j < LANES; ++j) t += red[j][ol];
+    out[o] = t;
+  }
 }
 
 __global__ void wgrad_reduce_kernel(const float *__restrict__ partial, int splits, long n,
@@ -957,6 +987,18 @@ int launch_readout_head(const occu_ctx *ctx, const DevCsr &csr, const float *h,
   return 1;
 }
 
+static int reduce_splits(const occu_ctx *ctx, const float *part, int splits, long n, float *out,
+                         cudaStream_t st) {
+  OCCU_PROF_BEGIN(ctx, "split_reduce", st);
+  if (n >= 4096)
+    split_reduce_kernel<8><<<int((n + 31) / 32), 256, 0, st>>>(part, splits, n, out);
+  else
+    split_reduce_kernel<64><<<int((n + 3) / 4), 256, 0, st>>>(part, splits, n, out);
+  OCCU_PROF_END(ctx);
+  LAUNCH_CHECK();
+  return 1;
+}
+
 static int wgrad(occu_ctx *ctx, const float *X, int A, const float *Y, int Bn, long R, float *out,
                  cudaStream_t st) {
   const long n = long(A) * Bn;
@@ -972,11 +1014,7 @@ static int wgrad(occu_ctx *ctx, const float *X, int A, const float *Y, int Bn, l
     float *part = ctx->ws.partial.as<float>();
     int r = launch_wgrad_tc(ctx, X, A, Y, Bn, R, sp, part, st);
     if (r < 0) return r;
-    OCCU_PROF_BEGIN(ctx, "wgrad_reduce", st);
-    wgrad_reduce_kernel<<<grid_for(n, 256, 1024), 256, 0, st>>>(part, sp, n, out);
-    OCCU_PROF_END(ctx);
-    LAUNCH_CHECK();
-    return r + 1;
+    return r + reduce_splits(ctx, part, sp, n, out, st);
   }
   if (n <= 2 * NT && A <= 128 && Bn <= 128) {
     const int sp = 2 * ctx->num_sms;
@@ -986,11 +1024,7 @@ static int wgrad(occu_ctx *ctx, const float *X, int A, const float *Y, int Bn, l
     wgrad_skinny_kernel<<<sp, NT, 0, st>>>(X, A, Y, Bn, R, sp, part);
     OCCU_PROF_END(ctx);
     LAUNCH_CHECK();
-    OCCU_PROF_BEGIN(ctx, "wgrad_reduce", st);
-    wgrad_reduce_kernel<<<grid_for(n, 256, 1024), 256, 0, st>>>(part, sp, n, out);
-    OCCU_PROF_END(ctx);
-    LAUNCH_CHECK();
-    return 2;
+    return 1 + reduce_splits(ctx, part, sp, n, out, st);
   }
   if (ctx->ws.partial.ensure(size_t(splits) * n * 4) != cudaSuccess) return -int(cudaErrorMemoryAllocation);
   float *part = ctx->ws.partial.as<float>();
@@ -1104,11 +1138,10 @@ static int backward_layer_impl(occu_ctx *ctx, const DevCsr &csr, const BwdLayerA
     LAUNCH_CHECK();
     ++n;
   }
-  const int nb_blocks = tc ? 2 * sms : grid_for(long(csr.N) * 32, NT, 16 * sms);
-  const int nb_warps = nb_blocks * (NT / 32);
+  const int nb_blocks = grid_for(long(csr.N) * 32, NT, 16 * sms);
   float *da_part = nullptr;
   if (tc) {
-    if (w.dpart.ensure(size_t(nb_warps) * 2 * D * 4) != cudaSuccess) return -int(cudaErrorMemoryAllocation);
+    if (w.dpart.ensure(size_t(nb_blocks) * 2 * D * 4) != cudaSuccess) return -int(cudaErrorMemoryAllocation);
     da_part = w.dpart.as<float>();
   }
   OCCU_PROF_BEGIN(ctx, "node_bwd", st);
@@ -1119,12 +1152,8 @@ static int backward_layer_impl(occu_ctx *ctx, const DevCsr &csr, const BwdLayerA
   LAUNCH_CHECK();
   ++n;
   if (tc) {
-    OCCU_PROF_BEGIN(ctx, "wgrad_reduce", st);
-    wgrad_reduce_kernel<<<grid_for(2 * D, 256, 1024), 256, 0, st>>>(da_part, nb_warps, 2 * D,
-                                                                     G + L.a_s[i]);
-    OCCU_PROF_END(ctx);
-    LAUNCH_CHECK();
-    ++n;
+    if ((r = reduce_splits(ctx, da_part, nb_blocks, 2 * D, G + L.a_s[i], st)) < 0) return r;
+    n += r;
   }
   // dW_m = DVᵀ E' ; dW_e = DZᵀ E_in ; dW_u = dPᵀ H_in ; [da_s; da_d] = [dp dq]ᵀ h̄
   if ((r = wgrad(ctx, w.DV.as<float>(), D, a.e, D, csr.E, G + L.W_m[i], st)) < 0) return r;
