@@ -48,6 +48,7 @@ constexpr int EPI_NODE = 0, EPI_EDGE = 1, EPI_GATE = 2;
 constexpr int EPI_PLAIN = 3;      // out = acc (+ add)
 constexpr int EPI_GATEBWD = 4;    // g = softmax(acc); dm = dA[t]; MG = dm ⊙ g; DV = g ⊙ (dm ⊙ h̄[s] - <g, dm ⊙ h̄[s]>)
 constexpr int EPI_EDGEBWD = 5;    // z = acc; dy = de ⊙ e' ⊙ σ(-αz); dα = <dy, z>; DZ = α dy
+constexpr int EPI_GATEAGG = 6;    // g = softmax(acc); m = g ⊙ h̄[s]; h[t] = LReLU(Σ_seg m) (a4-a6 fused)
 
 
 
@@ -81,6 +82,7 @@ struct RowGemmArgs {
   const int32_t *in_ptr;
   int mean;
   float *dal;              // EDGEBWD: dα [R]
+  float *part;             // GATEAGG: [R/32 units][2 slots][D] boundary-segment partials
 };
 
 struct Smem {
@@ -521,6 +523,98 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
             dot = hf == 0 ? dot + xg[128 + row] : xg[row] + dot;   // fixed order
           }
         }
+      } else if (EPI == EPI_GATEAGG) {
+        float m = -INFINITY;
+#pragma unroll
+        for (int c0 = 0; c0 < DH; c0 += 16) {
+          uint32_t r[16];
+          tc::tmem_ld16(acc + c0, r);
+          tc::tmem_ld_wait();
+#pragma unroll
+          for (int u = 0; u < 16; ++u) m = fmaxf(m, __uint_as_float(r[u]) * un);
+        }
+        xg[hf * 128 + row] = m;
+        group_bar(g);
+        m = fmaxf(m, xg[(hf ^ 1) * 128 + row]);
+        float sum = 0.f;
+#pragma unroll
+        for (int c0 = 0; c0 < DH; c0 += 16) {
+          uint32_t r[16];
+          tc::tmem_ld16(acc + c0, r);
+          tc::tmem_ld_wait();
+#pragma unroll
+          for (int u = 0; u < 16; ++u) sum += fast_exp(__uint_as_float(r[u]) * un - m);
+        }
+        xg[256 + hf * 128 + row] = sum;
+        group_bar(g);
+        sum = hf == 0 ? sum + xg[256 + 128 + row] : xg[256 + row] + sum;
+        const float inv = fast_rcp(sum);
+        // destination segments inside this warp's 32 consecutive (dst-sorted) edges
+        const int tn = live ? __ldg(a.dst + grow) : -1 - lane;         // pad rows: own segment
+        const int sn = live ? __ldg(a.src + grow) : 0;
+        const int tprev = __shfl_up_sync(0xffffffffu, tn, 1);
+        const int tnext = __shfl_down_sync(0xffffffffu, tn, 1);
+        const bool head = lane == 0 || tprev != tn;
+        const bool tail = lane == 31 || tnext != tn;
+        const unsigned heads = __ballot_sync(0xffffffffu, head);
+        const int start = 31 - __clz(heads & (0xffffffffu >> (31 - lane)));
+        int beg = 0, end = 0;
+        if (tail && live) {
+          beg = __ldg(a.in_ptr + tn);
+          end = __ldg(a.in_ptr + tn + 1);
+        }
+        const bool before = live && beg < wrow0 + start;               // segment began earlier
+        const bool after = live && end > wrow0 + lane + 1;               // continues after this warp
+        float dsc = 1.f;
+        if (a.mean) dsc = float(end - beg > 0 ? end - beg : 1);
+        const float *hbr = a.hbar + long(sn) * D + cb;
+        const long unit = wrow0 >> 5;
+#pragma unroll 1
+        for (int c0 = 0; c0 < DH; c0 += 16) {
+          uint32_t r[16];
+          tc::tmem_ld16(acc + c0, r);
+          tc::tmem_ld_wait();
+          float v[16];
+#pragma unroll
+          for (int u = 0; u < 16; u += 4) {
+            float4 b4 = make_float4(0.f, 0.f, 0.f, 0.f);
+            if (live) b4 = __ldg(reinterpret_cast<const float4 *>(hbr + c0 + u));
+            const float bv[4] = {b4.x, b4.y, b4.z, b4.w};
+#pragma unroll
+            for (int t = 0; t < 4; ++t)
+              v[u + t] = fast_exp(__uint_as_float(r[u + t]) * un - m) * inv * bv[t];   // m = g ⊙ h̄[s]
+          }
+          // segmented inclusive scan across lanes (fixed tree order)
+#pragma unroll
+          for (int d = 1; d < 32; d <<= 1) {
+#pragma unroll
+            for (int u = 0; u < 16; ++u) {
+              const float o = __shfl_up_sync(0xffffffffu, v[u], d);
+              if (lane - d >= start) v[u] += o;
+            }
+          }
+          if (tail && live) {
+            if (!before && !after) {                                   // complete segment
+              float *hr = a.out + long(tn) * D + cb + c0;
+#pragma unroll
+              for (int u = 0; u < 16; u += 4) {
+                float o4[4];
+#pragma unroll
+                for (int t = 0; t < 4; ++t) {
+                  float x = v[u + t];
+                  if (a.mean) x = x / dsc;
+                  o4[t] = lrelu(x, a.slope);
+                }
+                *reinterpret_cast<float4 *>(hr + u) = make_float4(o4[0], o4[1], o4[2], o4[3]);
+              }
+            } else {
+              float *pr = a.part + (unit * 2 + (before ? 0 : 1)) * D + cb + c0;
+#pragma unroll
+              for (int u = 0; u < 16; u += 4)
+                *reinterpret_cast<float4 *>(pr + u) = make_float4(v[u], v[u + 1], v[u + 2], v[u + 3]);
+            }
+          }
+        }
       } else if (EPI == EPI_GATE) {
         float m = -INFINITY;
 #pragma unroll
@@ -825,6 +919,41 @@ bool encode_rows_map(CUtensorMap *m, const float *A, int R, int K) {
             CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
 
+// Nodes whose in-edge segment spans several 32-edge units: combine the fixed-slot
+// partials in unit order; nodes without in-edges: h = LReLU(0) = 0 (R8).
+__global__ void agg_fixup_kernel(const int32_t *__restrict__ in_ptr, int N, int D,
+                                 const float *__restrict__ part, int mean, float slope,
+                                 float *__restrict__ h_out) {
+  const int warps = (gridDim.x * blockDim.x) / 32;
+  const int lane = threadIdx.x & 31;
+  for (int t0 = (blockIdx.x * blockDim.x + threadIdx.x) / 32 * 32; t0 < N; t0 += warps * 32) {
+    const int t = t0 + lane;
+    int beg = 0, end = 0;
+    if (t < N) {
+      beg = in_ptr[t];
+      end = in_ptr[t + 1];
+    }
+    const bool special = t < N && (beg == end || (beg >> 5) != ((end - 1) >> 5));
+    unsigned m = __ballot_sync(0xffffffffu, special);
+    while (m) {                                      // warp-cooperative over channels
+      const int l = __ffs(m) - 1;
+      m &= m - 1;
+      const int tt = t0 + l;
+      const int b2 = __shfl_sync(0xffffffffu, beg, l), e2 = __shfl_sync(0xffffffffu, end, l);
+      for (int c = lane; c < D; c += 32) {
+        float v = 0.f;
+        if (b2 != e2) {
+          const int ub = b2 >> 5, ue = (e2 - 1) >> 5;
+          v = part[(long(ub) * 2 + 1) * D + c];
+          for (int u = ub + 1; u <= ue; ++u) v += part[(long(u) * 2 + 0) * D + c];
+          if (mean) v = v / float(e2 - b2);
+        }
+        h_out[long(tt) * D + c] = lrelu(v, slope);
+      }
+    }
+  }
+}
+
 template <class Kern> void set_smem(Kern k, size_t bytes) {
   cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, int(bytes));
 }
@@ -879,7 +1008,7 @@ bool tc_supported(const occu_config &c) {
   return (c.d == 64 || c.d == 128) && c.F_n <= 128;
 }
 
-size_t tc_partial_floats(int E, int D) { return 16; }
+size_t tc_partial_floats(int E, int D) { return size_t(E / 32 + 2) * 2 * D; }
 
 template <int D, int EPI>
 static int launch_rowgemm(const occu_ctx *ctx, const RowGemmArgs &ra, const char *name,
@@ -900,7 +1029,7 @@ static int launch_rowgemm(const occu_ctx *ctx, const RowGemmArgs &ra, const char
 
 template <int D>
 static int tc_forward_layer_impl(const occu_ctx *ctx, const DevCsr &csr, const FwdLayerArgs &a,
-                                 cudaStream_t st) {
+                                 float *partial, cudaStream_t st) {
   const float slope = ctx->cfg.slope;
   int n = 0, r;
   RowGemmArgs ra{};
@@ -932,79 +1061,32 @@ static int tc_forward_layer_impl(const occu_ctx *ctx, const DevCsr &csr, const F
       if ((r = launch_rowgemm<D, EPI_EDGE>(ctx, re, "edge_tc", st)) < 0) return r;
       n += r;
     }
-    // a4: channel-softmax gate
+    // a4 + a5 + a6 fused: channel-softmax gate, message, segmented sum, LeakyReLU
     RowGemmArgs rg{};
     rg.slope = slope;
-    rg.A = a.e_out; rg.K = D; rg.R = csr.E; rg.W = a.W_m; rg.out = a.g;
-    if ((r = launch_rowgemm<D, EPI_GATE>(ctx, rg, "gate_tc", st)) < 0) return r;
+    rg.A = a.e_out; rg.K = D; rg.R = csr.E; rg.W = a.W_m; rg.out = a.h_out;
+    rg.hbar = a.hbar; rg.src = csr.in_src; rg.dst = csr.in_dst; rg.in_ptr = csr.in_ptr;
+    rg.mean = ctx->cfg.aggr == OCCU_AGGR_MEAN; rg.part = partial;
+    if ((r = launch_rowgemm<D, EPI_GATEAGG>(ctx, rg, "gate_agg_tc", st)) < 0) return r;
     n += r;
   }
-  // a5 + a6: gather + segmented sum (CUDA cores, warp per destination)
-  if ((r = launch_gather_segsum(ctx, csr, a.g, a.hbar, a.h_out, st)) < 0) return r;
-  return n + r;
-}
-
-// ---- backward row-GEMMs on tensor cores ------------------------------------
-template <int D>
-static int bwd_gate_impl(const occu_ctx *ctx, const DevCsr &csr, const float *e, const float *W_m,
-                         const float *dh, const float *h, const float *hbar, float *MG, float *DV,
-                         cudaStream_t st) {
-  RowGemmArgs r{};
-  r.slope = ctx->cfg.slope;
-  r.A = e; r.K = D; r.R = csr.E; r.W = W_m; r.out = MG; r.out2 = DV;
-  r.dh = dh; r.h = h; r.hbar = hbar; r.src = csr.in_src; r.dst = csr.in_dst;
-  r.in_ptr = csr.in_ptr; r.mean = ctx->cfg.aggr == OCCU_AGGR_MEAN;
-  return launch_rowgemm<D, EPI_GATEBWD>(ctx, r, "gate_bwd_tc", st);
-}
-template <int D>
-static int plain_impl(const occu_ctx *ctx, const float *A, int K, int R, const float *W, int transW,
-                      const float *add, float *out, const char *name, cudaStream_t st,
-                      const float *mask_h, const int32_t *in_ptr) {
-  RowGemmArgs r{};
-  r.slope = ctx->cfg.slope;
-  r.A = A; r.K = K; r.R = R; r.W = W; r.transW = transW; r.add = add; r.out = out;
-  r.mask_h = mask_h; r.in_ptr = in_ptr; r.mean = ctx->cfg.aggr == OCCU_AGGR_MEAN;
-  return launch_rowgemm<D, EPI_PLAIN>(ctx, r, name, st);
-}
-template <int D>
-static int bwd_edge_impl(const occu_ctx *ctx, const DevCsr &csr, const float *e_in, int Ke,
-                         const float *W_e, const float *e, const float *de, const float *p,
-                         const float *q, float *DZ, float *dal, cudaStream_t st) {
-  RowGemmArgs r{};
-  r.slope = ctx->cfg.slope;
-  r.A = e_in; r.K = Ke; r.R = csr.E; r.W = W_e; r.out = DZ; r.dal = dal;
-  r.e = e; r.de = de; r.pin = p; r.qin = q; r.src = csr.in_src; r.dst = csr.in_dst;
-  return launch_rowgemm<D, EPI_EDGEBWD>(ctx, r, "edge_bwd_tc", st);
-}
-
-int launch_bwd_gate_tc(const occu_ctx *ctx, const DevCsr &csr, const float *e, const float *W_m,
-                       const float *dh, const float *h, const float *hbar, float *MG, float *DV,
-                       cudaStream_t st) {
-  if (csr.E <= 0) return 0;
-  return ctx->cfg.d == 64 ? bwd_gate_impl<64>(ctx, csr, e, W_m, dh, h, hbar, MG, DV, st)
-                          : bwd_gate_impl<128>(ctx, csr, e, W_m, dh, h, hbar, MG, DV, st);
-}
-int launch_plain_tc(const occu_ctx *ctx, const float *A, int K, int R, const float *W, int transW,
-                    const float *add, float *out, const char *name, cudaStream_t st,
-                    const float *mask_h, const int32_t *in_ptr) {
-  if (R <= 0) return 0;
-  return ctx->cfg.d == 64 ? plain_impl<64>(ctx, A, K, R, W, transW, add, out, name, st, mask_h, in_ptr)
-                          : plain_impl<128>(ctx, A, K, R, W, transW, add, out, name, st, mask_h, in_ptr);
-}
-int launch_bwd_edge_tc(const occu_ctx *ctx, const DevCsr &csr, const float *e_in, int Ke,
-                       const float *W_e, const float *e, const float *de, const float *p,
-                       const float *q, float *DZ, float *dal, cudaStream_t st) {
-  if (csr.E <= 0) return 0;
-  return ctx->cfg.d == 64 ? bwd_edge_impl<64>(ctx, csr, e_in, Ke, W_e, e, de, p, q, DZ, dal, st)
-                          : bwd_edge_impl<128>(ctx, csr, e_in, Ke, W_e, e, de, p, q, DZ, dal, st);
+  if (csr.N > 0) {
+    const int grid = int(std::min<long>((long(csr.N) + 255) / 256, 8L * ctx->num_sms));
+    OCCU_PROF_BEGIN(ctx, "agg_fixup", st);
+    agg_fixup_kernel<<<grid, 256, 0, st>>>(csr.in_ptr, csr.N, D, partial,
+                                           ctx->cfg.aggr == OCCU_AGGR_MEAN, slope, a.h_out);
+    OCCU_PROF_END(ctx);
+    TC_CHECK();
+    ++n;
+  }
+  return n;
 }
 
 int launch_forward_layer_tc(const occu_ctx *ctx, const DevCsr &csr, const FwdLayerArgs &a,
                             float *partial, cudaStream_t st) {
-  (void)partial;
   switch (ctx->cfg.d) {
-    case 64: return tc_forward_layer_impl<64>(ctx, csr, a, st);
-    case 128: return tc_forward_layer_impl<128>(ctx, csr, a, st);
+    case 64: return tc_forward_layer_impl<64>(ctx, csr, a, partial, st);
+    case 128: return tc_forward_layer_impl<128>(ctx, csr, a, partial, st);
     default: return -int(cudaErrorInvalidValue);
   }
 }
