@@ -1082,6 +1082,61 @@ static int tc_forward_layer_impl(const occu_ctx *ctx, const DevCsr &csr, const F
   return n;
 }
 
+// ---- backward row-GEMMs on tensor cores ------------------------------------
+template <int D>
+static int bwd_gate_impl(const occu_ctx *ctx, const DevCsr &csr, const float *e, const float *W_m,
+                         const float *dh, const float *h, const float *hbar, float *MG, float *DV,
+                         cudaStream_t st) {
+  RowGemmArgs r{};
+  r.slope = ctx->cfg.slope;
+  r.A = e; r.K = D; r.R = csr.E; r.W = W_m; r.out = MG; r.out2 = DV;
+  r.dh = dh; r.h = h; r.hbar = hbar; r.src = csr.in_src; r.dst = csr.in_dst;
+  r.in_ptr = csr.in_ptr; r.mean = ctx->cfg.aggr == OCCU_AGGR_MEAN;
+  return launch_rowgemm<D, EPI_GATEBWD>(ctx, r, "gate_bwd_tc", st);
+}
+template <int D>
+static int plain_impl(const occu_ctx *ctx, const float *A, int K, int R, const float *W, int transW,
+                      const float *add, float *out, const char *name, cudaStream_t st,
+                      const float *mask_h, const int32_t *in_ptr) {
+  RowGemmArgs r{};
+  r.slope = ctx->cfg.slope;
+  r.A = A; r.K = K; r.R = R; r.W = W; r.transW = transW; r.add = add; r.out = out;
+  r.mask_h = mask_h; r.in_ptr = in_ptr; r.mean = ctx->cfg.aggr == OCCU_AGGR_MEAN;
+  return launch_rowgemm<D, EPI_PLAIN>(ctx, r, name, st);
+}
+template <int D>
+static int bwd_edge_impl(const occu_ctx *ctx, const DevCsr &csr, const float *e_in, int Ke,
+                         const float *W_e, const float *e, const float *de, const float *p,
+                         const float *q, float *DZ, float *dal, cudaStream_t st) {
+  RowGemmArgs r{};
+  r.slope = ctx->cfg.slope;
+  r.A = e_in; r.K = Ke; r.R = csr.E; r.W = W_e; r.out = DZ; r.dal = dal;
+  r.e = e; r.de = de; r.pin = p; r.qin = q; r.src = csr.in_src; r.dst = csr.in_dst;
+  return launch_rowgemm<D, EPI_EDGEBWD>(ctx, r, "edge_bwd_tc", st);
+}
+
+int launch_bwd_gate_tc(const occu_ctx *ctx, const DevCsr &csr, const float *e, const float *W_m,
+                       const float *dh, const float *h, const float *hbar, float *MG, float *DV,
+                       cudaStream_t st) {
+  if (csr.E <= 0) return 0;
+  return ctx->cfg.d == 64 ? bwd_gate_impl<64>(ctx, csr, e, W_m, dh, h, hbar, MG, DV, st)
+                          : bwd_gate_impl<128>(ctx, csr, e, W_m, dh, h, hbar, MG, DV, st);
+}
+int launch_plain_tc(const occu_ctx *ctx, const float *A, int K, int R, const float *W, int transW,
+                    const float *add, float *out, const char *name, cudaStream_t st,
+                    const float *mask_h, const int32_t *in_ptr) {
+  if (R <= 0) return 0;
+  return ctx->cfg.d == 64 ? plain_impl<64>(ctx, A, K, R, W, transW, add, out, name, st, mask_h, in_ptr)
+                          : plain_impl<128>(ctx, A, K, R, W, transW, add, out, name, st, mask_h, in_ptr);
+}
+int launch_bwd_edge_tc(const occu_ctx *ctx, const DevCsr &csr, const float *e_in, int Ke,
+                       const float *W_e, const float *e, const float *de, const float *p,
+                       const float *q, float *DZ, float *dal, cudaStream_t st) {
+  if (csr.E <= 0) return 0;
+  return ctx->cfg.d == 64 ? bwd_edge_impl<64>(ctx, csr, e_in, Ke, W_e, e, de, p, q, DZ, dal, st)
+                          : bwd_edge_impl<128>(ctx, csr, e_in, Ke, W_e, e, de, p, q, DZ, dal, st);
+}
+
 int launch_forward_layer_tc(const occu_ctx *ctx, const DevCsr &csr, const FwdLayerArgs &a,
                             float *partial, cudaStream_t st) {
   switch (ctx->cfg.d) {
