@@ -169,9 +169,11 @@ typedef enum {
   OCCU_T_R = 5,      /* [B][d]  readout */
   OCCU_T_YHAT = 6    /* [B] */
 } occu_tensor;
-/* Forward kernel path: 0 (default) = tcgen05 tensor cores, 3xTF32 split
- * products with FP32 accumulation in TMEM; 1 = CUDA-core FP32 (SIMT).  Both
- * meet the FP32 tolerance; the backward currently runs on CUDA cores. */
+/* Kernel path: 0 (default) = tcgen05 tensor cores (fp16x2-split GEMMs with
+ * per-row power-of-two scaling, FP32 accumulation in TMEM) + CUDA-core
+ * gather/segmented sum; 2 = as 0 with the gate, message and segmented sum fused
+ * into one tensor-core kernel; 1 = CUDA-core FP32 (SIMT) everywhere.  All meet
+ * the FP32 tolerance. */
 occu_status occu_set_kernel_path(occu_ctx *ctx, int path);
 /* Keep every intermediate of the next forward (costs memory/bandwidth). */
 occu_status occu_set_keep_intermediates(occu_ctx *ctx, int keep);

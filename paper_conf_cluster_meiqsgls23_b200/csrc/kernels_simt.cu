@@ -1008,7 +1008,7 @@ static int wgrad(occu_ctx *ctx, const float *X, int A, const float *Y, int Bn, l
     cudaMemsetAsync(out, 0, n * 4, st);
     return 0;
   }
-  if (ctx->path == 0 && wgrad_tc_supported(A, Bn) && R >= 4096) {
+  if (ctx->path != 1 && wgrad_tc_supported(A, Bn) && R >= 4096) {
     const int sp = ctx->num_sms;
     if (ctx->ws.partial.ensure(size_t(sp) * n * 4) != cudaSuccess) return -int(cudaErrorMemoryAllocation);
     float *part = ctx->ws.partial.as<float>();
@@ -1062,7 +1062,7 @@ int launch_head_backward(occu_ctx *ctx, const DevCsr &csr, const float *targets,
   OCCU_PROF_END(ctx);
   LAUNCH_CHECK();
   OCCU_PROF_BEGIN(ctx, "broadcast_dh", st);
-  const bool tcb = ctx->path == 0 && tc_supported(cf);    // TC backward consumes dA directly
+  const bool tcb = ctx->path != 1 && tc_supported(cf);    // TC backward consumes dA directly
   broadcast_dh_kernel<<<grid_for(long(csr.N) * cf.d, 256, 8192), 256, 0, st>>>(
       w.dr.as<float>(), csr.node_graph, csr.node_off, csr.N, cf.d,
       tcb ? w.h[cf.L - 1].as<float>() : nullptr, csr.in_ptr, cf.aggr == OCCU_AGGR_MEAN, cf.slope,
@@ -1084,7 +1084,7 @@ static int backward_layer_impl(occu_ctx *ctx, const DevCsr &csr, const BwdLayerA
   const int sms = ctx->num_sms;
   int n = 0;
   float *de = w.deA.as<float>();
-  const bool tc = ctx->path == 0 && tc_supported(cf);
+  const bool tc = ctx->path != 1 && tc_supported(cf);
   int r;
   if (tc && csr.E > 0) {
     // a10 on tensor cores: g recompute + softmax backward, W_mᵀ dv, z recompute + σ', W_eᵀ dz

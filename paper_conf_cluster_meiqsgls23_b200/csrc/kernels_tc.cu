@@ -558,6 +558,7 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
         const bool tail = lane == 31 || tnext != tn;
         const unsigned heads = __ballot_sync(0xffffffffu, head);
         const int start = 31 - __clz(heads & (0xffffffffu >> (31 - lane)));
+        const int maxlen = __reduce_max_sync(0xffffffffu, unsigned(lane - start + 1));
         int beg = 0, end = 0;
         if (tail && live) {
           beg = __ldg(a.in_ptr + tn);
@@ -585,8 +586,7 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
               v[u + t] = fast_exp(__uint_as_float(r[u + t]) * un - m) * inv * bv[t];   // m = g ⊙ h̄[s]
           }
           // segmented inclusive scan across lanes (fixed tree order)
-#pragma unroll
-          for (int d = 1; d < 32; d <<= 1) {
+          for (int d = 1; d < maxlen; d <<= 1) {        // only as many steps as the longest run
 #pragma unroll
             for (int u = 0; u < 16; ++u) {
               const float o = __shfl_up_sync(0xffffffffu, v[u], d);
@@ -1061,23 +1061,38 @@ static int tc_forward_layer_impl(const occu_ctx *ctx, const DevCsr &csr, const F
       if ((r = launch_rowgemm<D, EPI_EDGE>(ctx, re, "edge_tc", st)) < 0) return r;
       n += r;
     }
-    // a4 + a5 + a6 fused: channel-softmax gate, message, segmented sum, LeakyReLU
-    RowGemmArgs rg{};
-    rg.slope = slope;
-    rg.A = a.e_out; rg.K = D; rg.R = csr.E; rg.W = a.W_m; rg.out = a.h_out;
-    rg.hbar = a.hbar; rg.src = csr.in_src; rg.dst = csr.in_dst; rg.in_ptr = csr.in_ptr;
-    rg.mean = ctx->cfg.aggr == OCCU_AGGR_MEAN; rg.part = partial;
-    if ((r = launch_rowgemm<D, EPI_GATEAGG>(ctx, rg, "gate_agg_tc", st)) < 0) return r;
-    n += r;
+    if (ctx->path == 2) {
+      // a4 + a5 + a6 fused: channel-softmax gate, message, segmented sum, LeakyReLU
+      RowGemmArgs rg{};
+      rg.slope = slope;
+      rg.A = a.e_out; rg.K = D; rg.R = csr.E; rg.W = a.W_m; rg.out = a.h_out;
+      rg.hbar = a.hbar; rg.src = csr.in_src; rg.dst = csr.in_dst; rg.in_ptr = csr.in_ptr;
+      rg.mean = ctx->cfg.aggr == OCCU_AGGR_MEAN; rg.part = partial;
+      if ((r = launch_rowgemm<D, EPI_GATEAGG>(ctx, rg, "gate_agg_tc", st)) < 0) return r;
+      n += r;
+    } else {
+      // a4: channel-softmax gate -> g
+      RowGemmArgs rg{};
+      rg.slope = slope;
+      rg.A = a.e_out; rg.K = D; rg.R = csr.E; rg.W = a.W_m; rg.out = a.g;
+      if ((r = launch_rowgemm<D, EPI_GATE>(ctx, rg, "gate_tc", st)) < 0) return r;
+      n += r;
+    }
   }
-  if (csr.N > 0) {
-    const int grid = int(std::min<long>((long(csr.N) + 255) / 256, 8L * ctx->num_sms));
-    OCCU_PROF_BEGIN(ctx, "agg_fixup", st);
-    agg_fixup_kernel<<<grid, 256, 0, st>>>(csr.in_ptr, csr.N, D, partial,
-                                           ctx->cfg.aggr == OCCU_AGGR_MEAN, slope, a.h_out);
-    OCCU_PROF_END(ctx);
-    TC_CHECK();
-    ++n;
+  if (ctx->path == 2) {
+    if (csr.N > 0) {
+      const int grid = int(std::min<long>((long(csr.N) + 255) / 256, 8L * ctx->num_sms));
+      OCCU_PROF_BEGIN(ctx, "agg_fixup", st);
+      agg_fixup_kernel<<<grid, 256, 0, st>>>(csr.in_ptr, csr.N, D, partial,
+                                             ctx->cfg.aggr == OCCU_AGGR_MEAN, slope, a.h_out);
+      OCCU_PROF_END(ctx);
+      TC_CHECK();
+      ++n;
+    }
+  } else {
+    // a5 + a6: gather + segmented sum (CUDA cores, warp per 8 destinations)
+    if ((r = launch_gather_segsum(ctx, csr, a.g, a.hbar, a.h_out, st)) < 0) return r;
+    n += r;
   }
   return n;
 }

@@ -237,7 +237,7 @@ occu_status forward(occu_ctx *ctx, const DevCsr &csr, const float *nf, const flo
     a.e_out = (i < c.L - 1 || save_all) ? w.e[i].as<float>() : nullptr;
     a.g = w.g.as<float>();
     a.h_out = w.h[i].as<float>();
-    if (ctx->path == 0 && tc_supported(c)) {
+    if (ctx->path != 1 && tc_supported(c)) {
       a.e_out = w.e[i].as<float>();            // the gate kernel re-reads e'
       CK(w.tcpart.ensure(tc_partial_floats(csr.E, c.d) * 4), "alloc tc partials");
       LK(launch_forward_layer_tc(ctx, csr, a, w.tcpart.as<float>(), s), "forward layer (tc)");
@@ -641,7 +641,8 @@ occu_status occu_load_state(occu_ctx *ctx, const char *path) {
 
 occu_status occu_set_kernel_path(occu_ctx *ctx, int path) {
   if (!ctx) return fail(nullptr, OCCU_EINVAL, "ctx is NULL");
-  if (path != 0 && path != 1) return fail(ctx, OCCU_EINVAL, "path must be 0 (tensor cores) or 1 (SIMT)");
+  if (path < 0 || path > 2)
+    return fail(ctx, OCCU_EINVAL, "path must be 0 (tensor cores), 1 (SIMT) or 2 (tensor cores, fused aggregation)");
   ctx->path = path;
   return OCCU_OK;
 }

@@ -329,7 +329,8 @@ class Model:
         _check(lib().occu_dist_init(self._ctx, rank, world, buf), self._ctx)
 
     def set_kernel_path(self, path: int):
-        """0 = tensor cores (3xTF32, default), 1 = CUDA-core SIMT FP32."""
+        """0 = tensor cores (default), 1 = CUDA-core SIMT FP32, 2 = tensor cores with the
+        gate + aggregation fused."""
         _check(lib().occu_set_kernel_path(self._ctx, int(path)), self._ctx)
 
     # introspection

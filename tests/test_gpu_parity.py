@@ -69,7 +69,7 @@ def compare_all(m, c, y, ref, pk, tol=TOL):
     assert np.all(np.abs(y - yr) <= tol * np.maximum(np.abs(yr), 1e-2)), np.abs(y - yr).max()
 
 
-@pytest.mark.parametrize("path", [0, 1], ids=["tcgen05", "simt"])
+@pytest.mark.parametrize("path", [0, 1, 2], ids=["tcgen05", "simt", "tcgen05fused"])
 @pytest.mark.parametrize("L,d,aggr,seed", [(2, 64, 0, 1), (3, 128, 0, 2), (3, 128, 1, 3),
                                            (1, 64, 1, 4)])
 def test_random_batches_all_intermediates(L, d, aggr, seed, path):
@@ -80,7 +80,7 @@ def test_random_batches_all_intermediates(L, d, aggr, seed, path):
     compare_all(m, c, y, ref, pk)
 
 
-@pytest.mark.parametrize("path", [0, 1], ids=["tcgen05", "simt"])
+@pytest.mark.parametrize("path", [0, 1, 2], ids=["tcgen05", "simt", "tcgen05fused"])
 def test_hub_nodes_spanning_many_tiles(path):
     """Destination segments longer than a 128-edge tile (hubs) and ragged tails."""
     c = mk(2, 128)
@@ -152,7 +152,7 @@ def test_cfg2_full_size_sampled_graphs():
         assert abs(y[gi] - yr[0]) <= TOL * max(abs(yr[0]), 1e-2), gi
 
 
-@pytest.mark.parametrize("path", [0, 1], ids=["tcgen05", "simt"])
+@pytest.mark.parametrize("path", [0, 1, 2], ids=["tcgen05", "simt", "tcgen05fused"])
 def test_path_count_closed_form_bit_exact(path):
     """W_u = I, a = 0, W_m = 0, SUM, integer X >= 0 => H^i = (Aᵀ)^i X / d^i exactly."""
     d = 64
@@ -249,12 +249,14 @@ def test_errors():
 
 
 # ---------------------------------------------------------------- training
+@pytest.mark.parametrize("path", [0, 1], ids=["tcgen05", "simt"])
 @pytest.mark.parametrize("L,d,aggr", [(2, 64, 0), (3, 128, 0), (3, 128, 1)])
-def test_gradients_match_oracle(L, d, aggr):
+def test_gradients_match_oracle(L, d, aggr, path):
     c = mk(L, d, aggr=aggr)
     b = configs.random_dag_batch(24, 500 + L + aggr, max_nodes=50, hub=True)
     flat = weights.unit_scale(wcfg(c), weights.init_flat(wcfg(c), 11))
     m = occu.Model(c)
+    m.set_kernel_path(path)
     m.set_params(flat)
     loss = m.compute_grads(occu.pack(b.graphs), b.node_feat, b.edge_feat, b.targets)
     g = weights.unflatten(wcfg(c), m.get_grads())
