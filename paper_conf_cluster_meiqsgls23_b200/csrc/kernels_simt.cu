@@ -36,6 +36,15 @@ __device__ __forceinline__ float hsum16(float v) {   // sum over the 16 lanes sh
   v += __shfl_xor_sync(0xffffffffu, v, 8);
   return v;
 }
+// Cancellation-prone dot products (softmax backward <g, dg>, dα = <dy, z>) are
+// accumulated in float64 (a few hundred DFMA per edge).
+__device__ __forceinline__ double hsum16d(double v) {
+  v += __shfl_xor_sync(0xffffffffu, v, 1);
+  v += __shfl_xor_sync(0xffffffffu, v, 2);
+  v += __shfl_xor_sync(0xffffffffu, v, 4);
+  v += __shfl_xor_sync(0xffffffffu, v, 8);
+  return v;
+}
 __device__ __forceinline__ float hmax16(float v) {
   v = fmaxf(v, __shfl_xor_sync(0xffffffffu, v, 1));
   v = fmaxf(v, __shfl_xor_sync(0xffffffffu, v, 2));
@@ -548,16 +557,17 @@ __global__ void __launch_bounds__(NT) edge_bwd_m_kernel(
         const int deg = in_ptr[t + 1] - in_ptr[t];
         inv = float(deg > 0 ? deg : 1);
       }
-      float mg[TN], dg[TN], dot = 0.f;
+      float mg[TN], dg[TN];
+      double dotd = 0.0;
 #pragma unroll
       for (int j = 0; j < TN; ++j) {
         float dm = dhv[j] * lrelu_grad_from_out(hv[j], slope);
         if (mean) dm = dm / inv;
         dg[j] = dm * hb[j];
         mg[j] = dm * gg[j];
-        dot = fmaf(gg[j], dg[j], dot);
+        dotd = fma(double(gg[j]), double(dg[j]), dotd);
       }
-      dot = hsum16(dot);
+      const float dot = float(hsum16d(dotd));
 #pragma unroll
       for (int j = 0; j < TN; ++j) dv[i][j] = gg[j] * (dg[j] - dot);
       if (r < nrows) {
@@ -628,7 +638,8 @@ __global__ void __launch_bounds__(NT) edge_bwd_e_kernel(
 #pragma unroll
     for (int i = 0; i < 4; ++i) {
       const int r = ty * 4 + i;
-      float ev[TN], dev[TN], da = 0.f;
+      float ev[TN], dev[TN];
+      double dad = 0.0;
       if (r < nrows) {
         load_row<D>(e + (k0 + r) * D, ev, tx);
         load_row<D>(de + (k0 + r) * D, dev, tx);
@@ -642,10 +653,10 @@ __global__ void __launch_bounds__(NT) edge_bwd_e_kernel(
         // σ'(y) = σ(y)·σ(-y) with y = α z recomputed: avoids the cancellation of
         // 1 - e' when e' = σ(y) is close to 1 (float32).
         const float dyv = dev[j] * ev[j] * (1.f / (1.f + expf(al * acc[i][j])));
-        da = fmaf(dyv, acc[i][j], da);
+        dad = fma(double(dyv), double(acc[i][j]), dad);
         dz[i][j] = al * dyv;
       }
-      da = hsum16(da);
+      const float da = float(hsum16d(dad));
       if (r < nrows) {
         store_row<D>(DZ + (k0 + r) * D, dz[i], tx);
         if (tx == 0) dalpha[k0 + r] = da;

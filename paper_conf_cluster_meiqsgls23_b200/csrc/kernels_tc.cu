@@ -410,7 +410,7 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
           warp_store_chunk<D>(wbuf, a.out, wrow0, wrows, cb + c0, o, lane);
         }
       } else if (EPI == EPI_EDGEBWD) {
-        float dpart = 0.f;
+        double dpart = 0.0;                          // dα = <dy, z> in float64 (cancellation)
 #pragma unroll 1
         for (int c0 = 0; c0 < DH; c0 += 16) {
           uint32_t r[16];
@@ -431,15 +431,17 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
               const float z = __uint_as_float(r[u + t]) * un;
               // σ'(y) = σ(y)·σ(-y), y = α z (recomputed): no 1 - e' cancellation
               const float dy = dvv[t] * evv[t] * fast_rcp(1.f + fast_exp(aux * z));
-              dpart = fmaf(dy, z, dpart);
+              dpart = fma(double(dy), double(z), dpart);
               o[u + t] = aux * dy;
             }
           }
           warp_store_chunk<D>(wbuf, a.out, wrow0, wrows, cb + c0, o, lane);
         }
-        xg[256 + hf * 128 + row] = dpart;
+        double *xd = reinterpret_cast<double *>(xg);   // reuses the whole exchange area
+        group_bar(g);                                   // everyone has consumed the α slot
+        xd[hf * 128 + row] = dpart;
         group_bar(g);
-        if (hf == 0 && live) a.dal[grow] = dpart + xg[256 + 128 + row];
+        if (hf == 0 && live) a.dal[grow] = float(dpart + xd[128 + row]);
       } else if (EPI == EPI_GATEBWD) {
         // softmax statistics (as the forward gate)
         float m = -INFINITY;
@@ -478,6 +480,7 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
         }
         const float *dhr = a.dh + long(tn) * D + cb, *hr = is_dA ? dhr : a.h + long(tn) * D + cb;
         const float *hbr = a.hbar + long(sn) * D + cb;
+        double dotd = 0.0;     // <g, dg> in float64 (cancellation)
         float dot = 0.f;
         group_bar(g);          // everyone has read the (m, sum) exchange slots
 #pragma unroll 1
@@ -508,7 +511,7 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
                 }
                 const float dg = dm * bv[t];
                 if (pass == 0) {
-                  dot = fmaf(gg, dg, dot);
+                  dotd = fma(double(gg), double(dg), dotd);
                   o[u + t] = dm * gg;                              // MG
                 } else {
                   o[u + t] = gg * (dg - dot);                      // DV
@@ -518,9 +521,10 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
             warp_store_chunk<D>(wbuf, pass == 0 ? a.out : a.out2, wrow0, wrows, cb + c0, o, lane);
           }
           if (pass == 0) {
-            xg[hf * 128 + row] = dot;
+            double *xd = reinterpret_cast<double *>(xg);
+            xd[hf * 128 + row] = dotd;
             group_bar(g);
-            dot = hf == 0 ? dot + xg[128 + row] : xg[row] + dot;   // fixed order
+            dot = float(hf == 0 ? dotd + xd[128 + row] : xd[row] + dotd);   // fixed order
           }
         }
       } else if (EPI == EPI_GATEAGG) {
