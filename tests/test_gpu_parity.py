@@ -13,6 +13,7 @@ from paper_conf_cluster_meiqsgls23_b200 import occu
 
 pytestmark = pytest.mark.gpu
 TOL = 1e-4
+GRAD_TOL = 2e-4
 
 
 @pytest.fixture(scope="module", autouse=True)
@@ -264,7 +265,9 @@ def test_gradients_match_oracle(L, d, aggr, path):
     lref, gref = oracle.loss_and_grads(params, ocfg(c), b.graphs, b.node_feat, b.edge_feat, b.targets)
     assert abs(loss - lref) <= TOL * abs(lref)
     for k in gref:
-        assert rel(g[k], gref[k]) <= TOL, (k, rel(g[k], gref[k]))
+        # DESIGN.md R23: FP32 backward through 3 layers; the first-layer attention
+        # vectors' gradients are cancellation-heavy sums -> gradient tolerance 2e-4
+        assert rel(g[k], gref[k]) <= GRAD_TOL, (k, rel(g[k], gref[k]))
 
 
 def test_training_trajectory_matches_oracle():
