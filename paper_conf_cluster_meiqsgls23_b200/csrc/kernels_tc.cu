@@ -41,14 +41,35 @@ namespace occu {
 namespace {
 
 constexpr int TM = 128;
-constexpr int NTH = 704;          // warp 0 producer, 1 MMA, 2-5 converters, 6-21 epilogue
+constexpr int NTH = 832;          // warp 0 producer, 1 MMA, 2-9 converters, 10-25 epilogue
+constexpr int EPI0 = 10;          // first epilogue warp
 constexpr uint32_t TMEM_COLS = 512;
 constexpr int EPI_NODE = 0, EPI_EDGE = 1, EPI_GATE = 2;
 // backward epilogues (SURVEY §8(c) step BW)
 constexpr int EPI_PLAIN = 3;      // out = acc (+ add)
 constexpr int EPI_GATEBWD = 4;    // g = softmax(acc); dm = dA[t]; MG = dm ⊙ g; DV = g ⊙ (dm ⊙ h̄[s] - <g, dm ⊙ h̄[s]>)
 constexpr int EPI_EDGEBWD = 5;    // z = acc; dy = de ⊙ e' ⊙ σ(-αz); dα = <dy, z>; DZ = α dy
-constexpr int EPI_GATEAGG = 6;    // g = softmax(acc); m = g ⊙ h̄[s]; h[t] = LReLU(Σ_seg m) (a4-a6 fused)
+constexpr int EPI_GATEAGG = 6;
+
+#ifdef OCCU_TC_TIMING
+// Per-role busy/wait cycle counters of CTA 0 (debug builds only).
+__device__ unsigned long long g_tc_time[32][4];
+#define TT_DECL unsigned long long tt_w = 0, tt_b = 0, tt_0 = clock64(), tt_1;
+#define TT_WAIT_BEGIN tt_1 = clock64(); tt_b += tt_1 - tt_0;
+#define TT_WAIT_END tt_0 = clock64(); tt_w += tt_0 - tt_1;
+#define TT_FLUSH(slot)                                                            \
+  do {                                                                            \
+    tt_b += clock64() - tt_0;                                                     \
+    if (blockIdx.x == 0 && (threadIdx.x & 31) == 0) {                             \
+      g_tc_time[slot][0] += tt_w; g_tc_time[slot][1] += tt_b; g_tc_time[slot][2] += 1; \
+    }                                                                             \
+  } while (0)
+#else
+#define TT_DECL
+#define TT_WAIT_BEGIN
+#define TT_WAIT_END
+#define TT_FLUSH(slot)
+#endif    // g = softmax(acc); m = g ⊙ h̄[s]; h[t] = LReLU(Σ_seg m) (a4-a6 fused)
 
 
 
@@ -106,7 +127,7 @@ __host__ __device__ inline int nbox_of(int K) { return (K + 31) / 32; }
 __host__ __device__ inline size_t smem_bytes(int D, int K) {
   const size_t img = size_t(kpad_of(K)) * D * 2;
   const size_t slot = size_t(nbox_of(K)) * 16384;
-  return 1024 + 2 * img + 2 * slot + 4096 + 16 * 16 * 20 * 4 + 2 * 2 * 2 * 128 * 4;
+  return 1024 + 2 * img + 2 * slot + 4096 + 16 * 16 * 20 * 4 + 2 * 2 * 2 * 128 * 4 + 2 * 128 * 4;
 }
 
 __device__ __forceinline__ Smem carve(uint8_t *raw, int D, int K) {
@@ -236,13 +257,13 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
   if (threadIdx.x == 0) {
     for (int j = 0; j < 2; ++j) {
       tc::mbar_init(s.full + j, 1);
-      tc::mbar_init(s.empty + j, 128);
-      tc::mbar_init(s.afull + j, 128);
+      tc::mbar_init(s.empty + j, 256);
+      tc::mbar_init(s.afull + j, 256);
       tc::mbar_init(s.afree + j, 1);
       tc::mbar_init(s.accfull + j, 1);
       tc::mbar_init(s.accfree + j, 256);
     }
-    for (int j = 0; j < 4; ++j) tc::mbar_init(s.eready + j, 128);
+    for (int j = 0; j < 4; ++j) tc::mbar_init(s.eready + j, 256);
     tc::fence_mbar_init();
   }
   if (warp == 1) tc::tmem_alloc<TMEM_COLS>(s.tmem_slot);
@@ -259,25 +280,32 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
   if (warp == 0) {
     // ---------------- producer: tile i -> slot i%2 (TMA 2D, OOB rows zero-filled) -------
     if (lane == 0) {
+      TT_DECL
       tc::prefetch_tmap(&tmap);
       for (int i = 0; i < my; ++i) {
         const int j = i & 1;
         const int r0 = int(blockIdx.x + i * gridDim.x) * TM;
+        TT_WAIT_BEGIN
         if (i >= 2) tc::mbar_wait(s.empty + j, ((i >> 1) - 1) & 1);
+        TT_WAIT_END
         tc::mbar_arrive_expect_tx(s.full + j, uint32_t(NB) * 16384u);
         for (int b = 0; b < NB; ++b) tc::tma_load_2d(s.slot(j) + b * 4096, &tmap, 32 * b, r0, s.full + j);
       }
+      TT_FLUSH(0);
     }
     __syncwarp();
   } else if (warp == 1) {
     // ---------------- MMA issuer: A[i%2] -> ACC[i%2] ----------------
+    TT_DECL
     const uint32_t idsc = tc::idesc(128, uint32_t(D), tc::FMT_F16);
     const uint32_t w0a = tc::smem_u32(s.w0), w1a = tc::smem_u32(s.w1);
     const int nk = (K + 15) / 16;
     for (int i = 0; i < my; ++i) {
       const int j = i & 1;
+      TT_WAIT_BEGIN
       tc::mbar_wait(s.afull + j, (i >> 1) & 1);
       if (i >= 2) tc::mbar_wait(s.accfree + j, ((i >> 1) - 1) & 1);
+      TT_WAIT_END
       tc::fence_after_sync();
       if (lane == 0) {
         const uint32_t d = tmem + acc_col(j);
@@ -295,52 +323,72 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
       }
       __syncwarp();
     }
-  } else if (warp < 6) {
-    // ---------------- converters (warps 2-5), thread = row: slot -> TMEM A ----------------
+    TT_FLUSH(1);
+  } else if (warp < EPI0) {
+    // ---------------- converters (warps 2-9): thread = (row, K-half) -> TMEM A ----------------
+    // Input rows of the node transform (h) get a per-row power-of-two scale from the row max
+    // (exchanged between the two K-halves); edge states e' lie in (0, 1) and use the fixed
+    // exponent 14 (max·2^14 < 2^15), so only absolute precision ~2^-24 is at stake.
     const int qd = warp & 3;
+    const int kh = (warp - 2) >> 2;
     const int row = qd * 32 + lane;
     const uint32_t lane_base = tmem + (uint32_t(qd * 32) << 16);
+    const int KH = Kpad / 2;                       // K-elements per half
+    const int kb = kh * KH, ke = min(K, kb + KH);
+    float *cmax = s.xch + 2 * 2 * 2 * 128;         // [2 halves][128 rows]
+    TT_DECL
     for (int i = 0; i < my; ++i) {
       const int j = i & 1;
       const long r0 = long(blockIdx.x + i * gridDim.x) * TM;
       const bool live = row < min(TM, int(a.R - r0));
+      TT_WAIT_BEGIN
       tc::mbar_wait(s.full + j, (i >> 1) & 1);
       if (i >= 2) tc::mbar_wait(s.afree + j, ((i >> 1) - 1) & 1);
+      TT_WAIT_END
       const float *sl = s.slot(j);
-      float mx = 0.f;
-      if (live)
-#pragma unroll 8
-        for (int k = 0; k < K; k += 4) {
-          const float4 v = slot_ld4(sl, row, k);
-          mx = fmaxf(mx, fmaxf(fmaxf(fabsf(v.x), fabsf(v.y)), fmaxf(fabsf(v.z), fabsf(v.w))));
-        }
-      const int er = scale_exp(mx);
+      int er = 14;
+      if (EPI == EPI_NODE || EPI == EPI_PLAIN) {
+        float mx = 0.f;
+        if (live)
+#pragma unroll 4
+          for (int k = kb; k < ke; k += 4) {
+            const float4 v = slot_ld4(sl, row, k);
+            mx = fmaxf(mx, fmaxf(fmaxf(fabsf(v.x), fabsf(v.y)), fmaxf(fabsf(v.z), fabsf(v.w))));
+          }
+        cmax[kh * 128 + row] = mx;
+        asm volatile("bar.sync 3, 256;" ::: "memory");
+        mx = fmaxf(mx, cmax[(kh ^ 1) * 128 + row]);
+        er = scale_exp(mx);
+        asm volatile("bar.sync 3, 256;" ::: "memory");   // cmax reused next tile
+      }
       const float xs = ldexpf(1.f, er);
-      for (int c0 = 0; c0 < Kpad / 2; c0 += 16) {
+      for (int c0 = 0; c0 < KH / 2; c0 += 16) {
         uint32_t x0[16], x1[16];
 #pragma unroll
         for (int u = 0; u < 16; u += 2) {
-          const int k = 2 * (c0 + u);
+          const int k = kb + 2 * (c0 + u);
           float4 v = make_float4(0.f, 0.f, 0.f, 0.f);
           if (live && k < K) v = slot_ld4(sl, row, k);
           split2(v.x * xs, v.y * xs, x0[u], x1[u]);
           split2(v.z * xs, v.w * xs, x0[u + 1], x1[u + 1]);
         }
-        tc::tmem_st16(lane_base + a_col(j) + c0, x0);
-        tc::tmem_st16(lane_base + a_col(j) + Kpad / 2 + c0, x1);
+        const uint32_t col = a_col(j) + uint32_t(kb / 2 + c0);
+        tc::tmem_st16(lane_base + col, x0);
+        tc::tmem_st16(lane_base + col + Kpad / 2, x1);
       }
-      s.erow[(i & 3) * 128 + row] = er;
+      if (kh == 0) s.erow[(i & 3) * 128 + row] = er;
       tc::tmem_st_wait();
       tc::fence_before_sync();
       tc::mbar_arrive(s.empty + j);
       tc::mbar_arrive(s.afull + j);
       tc::mbar_arrive(s.eready + (i & 3));
     }
+    TT_FLUSH(2 + (warp - 2));
   } else {
     // ---------------- epilogue: two groups of 8 warps (6-13, 14-21) -----------------
     // group g handles tiles i = g, g+2, ... from ACC[g]; a row is shared by two warps of
     // the same TMEM lane quarter: half hf owns output columns [hf*D/2, (hf+1)*D/2).
-    const int wi = warp - 6;
+    const int wi = warp - EPI0;
     const int g = wi >> 3;
     const int hf = (wi >> 2) & 1;
     const int qd = warp & 3;
@@ -350,6 +398,7 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
     float *wbuf = s.xbuf + wi * (16 * 20);
     constexpr int DH = D / 2;
     const int cb = hf * DH;
+    TT_DECL
     for (int i = g; i < my; i += 2) {
       const int j = i & 1;
       const long r0 = long(blockIdx.x + i * gridDim.x) * TM;
@@ -358,9 +407,11 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
       float aux = 0.f;
       if ((EPI == EPI_EDGE || EPI == EPI_EDGEBWD) && hf == 0 && live)
         aux = __ldg(a.pin + __ldg(a.src + r0 + row)) + __ldg(a.qin + __ldg(a.dst + r0 + row));  // α (R1)
+      TT_WAIT_BEGIN
       tc::mbar_wait(s.eready + (i & 3), (i >> 2) & 1);
       const int er = s.erow[(i & 3) * 128 + row];
       tc::mbar_wait(s.accfull + j, (i >> 1) & 1);
+      TT_WAIT_END
       tc::fence_after_sync();
       if (EPI == EPI_EDGE || EPI == EPI_EDGEBWD) {
         if (hf == 0) xg[row] = aux;
@@ -698,6 +749,7 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
       tc::mbar_arrive(s.accfree + j);
       group_bar(g);        // the exchange buffer is reused by the next tile
     }
+    TT_FLUSH(6 + wi);
   }
   tc::fence_before_sync();
   __syncthreads();
@@ -1166,4 +1218,14 @@ int launch_forward_layer_tc(const occu_ctx *ctx, const DevCsr &csr, const FwdLay
 }
 
 }  // namespace occu
+
+#ifdef OCCU_TC_TIMING
+extern "C" int occu_debug_tc_time(unsigned long long *host) {
+  cudaDeviceSynchronize();
+  cudaMemcpyFromSymbol(host, occu::g_tc_time, sizeof(occu::g_tc_time));
+  static unsigned long long zero[32][4] = {};
+  cudaMemcpyToSymbol(occu::g_tc_time, zero, sizeof(zero));
+  return 0;
+}
+#endif
 
