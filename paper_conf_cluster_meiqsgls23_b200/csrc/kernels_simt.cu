@@ -1099,14 +1099,14 @@ static int backward_layer_impl(occu_ctx *ctx, const DevCsr &csr, const BwdLayerA
   int r;
   if (tc && csr.E > 0) {
     // a10 on tensor cores: g recompute + softmax backward, W_mᵀ dv, z recompute + σ', W_eᵀ dz
-    if ((r = launch_bwd_gate_tc(ctx, csr, a.e, P + L.W_m[i], a.dh, nullptr, a.hbar, w.MG.as<float>(),
+    if ((r = launch_bwd_gate_tc(ctx, csr, i, a.e, a.dh, nullptr, a.hbar, w.MG.as<float>(),
                                 w.DV.as<float>(), st)) < 0) return r;
     n += r;
-    if ((r = launch_plain_tc(ctx, w.DV.as<float>(), D, csr.E, P + L.W_m[i], 1, a.de_out, de,
+    if ((r = launch_plain_tc(ctx, w.DV.as<float>(), D, csr.E, 3, i, a.de_out, de,
                              "de_tc", st)) < 0) return r;
     n += r;
     if (a.Ke > 16) {
-      if ((r = launch_bwd_edge_tc(ctx, csr, a.e_in, a.Ke, P + L.W_e[i], a.e, de, a.p, a.q,
+      if ((r = launch_bwd_edge_tc(ctx, csr, i, a.e_in, a.Ke, a.e, de, a.p, a.q,
                                   w.DZ.as<float>(), w.dalpha.as<float>(), st)) < 0) return r;
       n += r;
     } else {
@@ -1123,7 +1123,7 @@ static int backward_layer_impl(occu_ctx *ctx, const DevCsr &csr, const BwdLayerA
       ++n;
     }
     if (a.de_prev) {
-      if ((r = launch_plain_tc(ctx, w.DZ.as<float>(), D, csr.E, P + L.W_e[i], 1, nullptr,
+      if ((r = launch_plain_tc(ctx, w.DZ.as<float>(), D, csr.E, 4, i, nullptr,
                                a.de_prev, "de_prev_tc", st)) < 0) return r;
       n += r;
     }
@@ -1178,7 +1178,7 @@ static int backward_layer_impl(occu_ctx *ctx, const DevCsr &csr, const BwdLayerA
     n += r;
   }
   if (a.dh_prev && csr.N > 0 && tc) {   // dh^{i-1} = dP W_u on tensor cores
-    if ((r = launch_plain_tc(ctx, w.dP.as<float>(), D, csr.N, P + L.W_u[i], 1, nullptr, a.dh_prev,
+    if ((r = launch_plain_tc(ctx, w.dP.as<float>(), D, csr.N, 5, i, nullptr, a.dh_prev,
                              "dh_prev_tc", st, a.h_in, csr.in_ptr)) < 0) return r;
     n += r;
   } else if (a.dh_prev && csr.N > 0) {   // dh^{i-1} = dP W_u  (K == D for i > 0)
@@ -1206,6 +1206,7 @@ int launch_backward_layer(occu_ctx *ctx, const DevCsr &csr, const BwdLayerArgs &
 }
 
 int launch_adam(occu_ctx *ctx, float lr, cudaStream_t st) {
+  ctx->params_version += 1;        // tensor-core weight images must be rebuilt
   const long n = long(ctx->layout.total);
   const double b1 = 0.9, b2 = 0.999;
   const double bc1 = 1.0 - pow(b1, double(ctx->adam_t));

@@ -33,6 +33,7 @@
 
 #include <algorithm>
 #include <cstdlib>
+#include <vector>
 
 #include "occu_internal.h"
 #include "tc_common.cuh"
@@ -88,7 +89,9 @@ __device__ __forceinline__ float fast_rcp(float x) {
 struct RowGemmArgs {
   const float *A;          // [R][K] input rows (fp32)
   int K, R;
-  const float *W;          // [D][K]
+  const float *W;          // [D][K] (unused by the kernel: see wimg)
+  const uint8_t *wimg;     // prebuilt fp16x2 SW128 images of W: [w0 | w1], Kpad*D*2 bytes each
+  const int *wfexp;        // weight scale exponent f
   float *out;              // [R][D]
   const float *a_s, *a_d;  // NODE
   float *p, *q;            // NODE outputs
@@ -111,7 +114,7 @@ struct Smem {
   float *slot0;
   int slot_floats;
   __device__ __forceinline__ float *slot(int j) const { return slot0 + j * slot_floats; }
-  uint64_t *full, *empty, *afull, *afree, *accfull, *accfree, *eready;
+  uint64_t *full, *empty, *afull, *afree, *accfull, *accfree, *eready, *wfull;
   uint32_t *tmem_slot;
   int *fexp;
   float *red;
@@ -149,8 +152,9 @@ __device__ __forceinline__ Smem carve(uint8_t *raw, int D, int K) {
   s.accfull = bars + 8;
   s.accfree = bars + 10;
   s.eready = bars + 12;                 // 4
-  s.tmem_slot = reinterpret_cast<uint32_t *>(misc + 128);
-  s.fexp = reinterpret_cast<int *>(misc + 132);
+  s.wfull = bars + 16;
+  s.tmem_slot = reinterpret_cast<uint32_t *>(misc + 144);
+  s.fexp = reinterpret_cast<int *>(misc + 148);
   s.red = reinterpret_cast<float *>(misc + 256);
   s.avec = reinterpret_cast<float *>(misc + 512);
   s.erow = reinterpret_cast<int *>(misc + 1536);
@@ -218,37 +222,15 @@ template <int D, int EPI>
 __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__ CUtensorMap tmap,
                                                          RowGemmArgs a) {
   extern __shared__ uint8_t smem_raw[];
+#ifdef OCCU_TC_TIMING
+  const unsigned long long t_entry = clock64();
+#endif
   const int K = a.K, Kpad = kpad_of(K), NB = nbox_of(K);
   Smem s = carve(smem_raw, D, K);
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
 
-  // ---- weight scale 2^f (block max |W|) and fp16x2 SW128 images ------------
-  float wmx = 0.f;
-  for (int i = threadIdx.x; i < D * K; i += NTH) wmx = fmaxf(wmx, fabsf(__ldg(a.W + i)));   // any layout
-#pragma unroll
-  for (int o = 16; o > 0; o >>= 1) wmx = fmaxf(wmx, __shfl_xor_sync(0xffffffffu, wmx, o));
-  if (lane == 0) s.red[warp] = wmx;
-  __syncthreads();
-  if (threadIdx.x == 0) {
-    float m = 0.f;
-    for (int w = 0; w < NTH / 32; ++w) m = fmaxf(m, s.red[w]);
-    *s.fexp = scale_exp(m);
-  }
-  __syncthreads();
-  const int fexp = *s.fexp;
-  const float wscale = ldexpf(1.f, fexp);
-  for (int i = threadIdx.x; i < D * (Kpad / 2); i += NTH) {
-    const int n = i / (Kpad / 2), k = 2 * (i % (Kpad / 2));
-    const long i0 = a.transW ? long(k) * D + n : long(n) * K + k;
-    const long i1 = a.transW ? long(k + 1) * D + n : long(n) * K + k + 1;
-    const float v0 = k < K ? __ldg(a.W + i0) * wscale : 0.f;
-    const float v1 = k + 1 < K ? __ldg(a.W + i1) * wscale : 0.f;
-    uint32_t hi, lo;
-    split2(v0, v1, hi, lo);
-    const uint32_t off = tc::sw128_offset_f16(n, k, D);
-    *reinterpret_cast<uint32_t *>(s.w0 + off) = hi;
-    *reinterpret_cast<uint32_t *>(s.w1 + off) = lo;
-  }
+  // ---- weights: prebuilt fp16x2 images (wimage_kernel), bulk-copied by the producer ----
+  const int fexp = __ldg(a.wfexp);
   if (EPI == EPI_NODE)
     for (int i = threadIdx.x; i < D; i += NTH) {
       s.avec[i] = a.a_s[i];
@@ -264,6 +246,7 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
       tc::mbar_init(s.accfree + j, 256);
     }
     for (int j = 0; j < 4; ++j) tc::mbar_init(s.eready + j, 256);
+    tc::mbar_init(s.wfull, 1);
     tc::fence_mbar_init();
   }
   if (warp == 1) tc::tmem_alloc<TMEM_COLS>(s.tmem_slot);
@@ -273,6 +256,12 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
   __syncthreads();
   tc::fence_after_sync();
   const uint32_t tmem = *s.tmem_slot;
+#ifdef OCCU_TC_TIMING
+  if (blockIdx.x == 0 && threadIdx.x == 0) {
+    g_tc_time[30][1] += clock64() - t_entry;
+    g_tc_time[30][2] += 1;
+  }
+#endif
 
   const int tiles = (a.R + TM - 1) / TM;
   const int my = blockIdx.x < tiles ? (tiles - 1 - int(blockIdx.x)) / int(gridDim.x) + 1 : 0;
@@ -282,6 +271,15 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
     if (lane == 0) {
       TT_DECL
       tc::prefetch_tmap(&tmap);
+      {   // weight images -> smem (16 KB bulk copies)
+        const uint32_t ib = uint32_t(Kpad) * D * 2;
+        tc::mbar_arrive_expect_tx(s.wfull, 2 * ib);
+        for (uint32_t o = 0; o < ib; o += 16384) {
+          const uint32_t n = ib - o < 16384 ? ib - o : 16384;
+          tc::bulk_g2s(s.w0 + o, a.wimg + o, n, s.wfull);
+          tc::bulk_g2s(s.w1 + o, a.wimg + ib + o, n, s.wfull);
+        }
+      }
       for (int i = 0; i < my; ++i) {
         const int j = i & 1;
         const int r0 = int(blockIdx.x + i * gridDim.x) * TM;
@@ -300,6 +298,7 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
     const uint32_t idsc = tc::idesc(128, uint32_t(D), tc::FMT_F16);
     const uint32_t w0a = tc::smem_u32(s.w0), w1a = tc::smem_u32(s.w1);
     const int nk = (K + 15) / 16;
+    tc::mbar_wait(s.wfull, 0);
     for (int i = 0; i < my; ++i) {
       const int j = i & 1;
       TT_WAIT_BEGIN
@@ -749,12 +748,64 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
       tc::mbar_arrive(s.accfree + j);
       group_bar(g);        // the exchange buffer is reused by the next tile
     }
-    TT_FLUSH(6 + wi);
+    TT_FLUSH(10 + wi);
   }
   tc::fence_before_sync();
   __syncthreads();
   tc::fence_after_sync();
   if (warp == 1) tc::tmem_dealloc<TMEM_COLS>(tmem);
+#ifdef OCCU_TC_TIMING
+  if (blockIdx.x == 0 && threadIdx.x == 0) {
+    g_tc_time[31][1] += clock64() - t_entry;
+    g_tc_time[31][2] += 1;
+  }
+#endif
+}
+
+// ---------------------------------------------------------------------------
+// Weight images (built once per parameter update, shared by every row-GEMM launch):
+// scale exponent f (max |W|·2^f in [2^14, 2^15)), W·2^f split into fp16 hi / lo in the
+// SW128 K-major B-operand layout, [w0 | w1].  One CTA per matrix.
+// ---------------------------------------------------------------------------
+struct WImageJob {
+  const float *W;
+  int D, K, transW;
+  uint8_t *img;
+  int *fexp;
+};
+
+__global__ void __launch_bounds__(256) wimage_kernel(const WImageJob *__restrict__ jobs) {
+  const WImageJob jb = jobs[blockIdx.x];
+  const int D = jb.D, K = jb.K, Kpad = kpad_of(K);
+  __shared__ float red[8];
+  __shared__ int fe;
+  float m = 0.f;
+  for (int i = threadIdx.x; i < D * K; i += 256) m = fmaxf(m, fabsf(jb.W[i]));
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, o));
+  if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = m;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    float mm = 0.f;
+    for (int w = 0; w < 8; ++w) mm = fmaxf(mm, red[w]);
+    fe = scale_exp(mm);
+    *jb.fexp = fe;
+  }
+  __syncthreads();
+  const float ws = ldexpf(1.f, fe);
+  const uint32_t ib = uint32_t(Kpad) * D * 2;
+  for (int i = threadIdx.x; i < D * (Kpad / 2); i += 256) {
+    const int n = i / (Kpad / 2), k = 2 * (i % (Kpad / 2));
+    const long i0 = jb.transW ? long(k) * D + n : long(n) * K + k;
+    const long i1 = jb.transW ? long(k + 1) * D + n : long(n) * K + k + 1;
+    const float v0 = k < K ? jb.W[i0] * ws : 0.f;
+    const float v1 = k + 1 < K ? jb.W[i1] * ws : 0.f;
+    uint32_t hi, lo;
+    split2(v0, v1, hi, lo);
+    const uint32_t off = tc::sw128_offset_f16(n, k, D);
+    *reinterpret_cast<uint32_t *>(jb.img + off) = hi;
+    *reinterpret_cast<uint32_t *>(jb.img + ib + off) = lo;
+  }
 }
 
 // Layer-1 edge transform (F_e small, e.g. 4): e' = σ(α · W_e e) on CUDA cores,
@@ -1060,6 +1111,55 @@ int launch_wgrad_tc(const occu_ctx *ctx, const float *X, int A, const float *Y, 
   return 1;
 }
 
+constexpr size_t WIMG_MAX = size_t(2) * 128 * 128 * 2;   // [w0 | w1], Kpad <= 128, D <= 128
+
+const uint8_t *tc_wimg(const occu_ctx *ctx, int kind, int layer) {
+  return ctx->wimg.as<uint8_t>() + size_t(layer * 6 + kind) * WIMG_MAX;
+}
+const int *tc_wfexp(const occu_ctx *ctx, int kind, int layer) {
+  return ctx->wfexp.as<int>() + layer * 6 + kind;
+}
+
+// (Re)build the images when the parameters changed (set_params / Adam bump the version).
+int tc_prepare_weights(occu_ctx *ctx, cudaStream_t st) {
+  if (ctx->wimg_version == ctx->params_version) return 0;
+  const occu_config &c = ctx->cfg;
+  const ParamLayout &L = ctx->layout;
+  if (ctx->wimg.ensure(size_t(c.L) * 6 * WIMG_MAX) != cudaSuccess ||
+      ctx->wfexp.ensure(size_t(c.L) * 6 * sizeof(int)) != cudaSuccess ||
+      ctx->wjobs.ensure(size_t(c.L) * 6 * sizeof(WImageJob)) != cudaSuccess)
+    return -int(cudaErrorMemoryAllocation);
+  std::vector<WImageJob> jobs;
+  const float *P = ctx->params.as<float>();
+  for (int i = 0; i < c.L; ++i) {
+    auto add = [&](int kind, const float *W, int D, int K, int transW) {
+      WImageJob j;
+      j.W = W; j.D = D; j.K = K; j.transW = transW;
+      j.img = const_cast<uint8_t *>(tc_wimg(ctx, kind, i));
+      j.fexp = const_cast<int *>(tc_wfexp(ctx, kind, i));
+      jobs.push_back(j);
+    };
+    if (L.d_in[i] <= 128) add(0, P + L.W_u[i], c.d, L.d_in[i], 0);
+    if (L.de_in[i] > 16 && L.de_in[i] <= 128) {
+      add(1, P + L.W_e[i], c.d, L.de_in[i], 0);
+      add(4, P + L.W_e[i], c.d, c.d, 1);
+    }
+    add(2, P + L.W_m[i], c.d, c.d, 0);
+    add(3, P + L.W_m[i], c.d, c.d, 1);
+    if (i > 0) add(5, P + L.W_u[i], c.d, c.d, 1);
+  }
+  // job table: pointers are fixed for the ctx, re-uploaded only with the images
+  if (cudaMemcpyAsync(ctx->wjobs.ptr, jobs.data(), jobs.size() * sizeof(WImageJob),
+                      cudaMemcpyHostToDevice, st) != cudaSuccess)
+    return -int(cudaErrorInvalidValue);
+  OCCU_PROF_BEGIN(ctx, "wimage", st);
+  wimage_kernel<<<int(jobs.size()), 256, 0, st>>>(ctx->wjobs.as<WImageJob>());
+  OCCU_PROF_END(ctx);
+  TC_CHECK();
+  ctx->wimg_version = ctx->params_version;
+  return 1;
+}
+
 bool tc_supported(const occu_config &c) {
   return (c.d == 64 || c.d == 128) && c.F_n <= 128;
 }
@@ -1084,14 +1184,15 @@ static int launch_rowgemm(const occu_ctx *ctx, const RowGemmArgs &ra, const char
 }
 
 template <int D>
-static int tc_forward_layer_impl(const occu_ctx *ctx, const DevCsr &csr, const FwdLayerArgs &a,
-                                 float *partial, cudaStream_t st) {
+static int tc_forward_layer_impl(const occu_ctx *ctx, const DevCsr &csr, int layer,
+                                 const FwdLayerArgs &a, float *partial, cudaStream_t st) {
   const float slope = ctx->cfg.slope;
   int n = 0, r;
   RowGemmArgs ra{};
   ra.slope = slope;
   // a2: node transform
   ra.A = a.h_in; ra.K = a.K; ra.R = csr.N; ra.W = a.W_u; ra.out = a.hbar;
+  ra.wimg = tc_wimg(ctx, 0, layer); ra.wfexp = tc_wfexp(ctx, 0, layer);
   ra.a_s = a.a_s; ra.a_d = a.a_d; ra.p = a.p; ra.q = a.q;
   if ((r = launch_rowgemm<D, EPI_NODE>(ctx, ra, "node_tc", st)) < 0) return r;
   n += r;
@@ -1113,6 +1214,7 @@ static int tc_forward_layer_impl(const occu_ctx *ctx, const DevCsr &csr, const F
       RowGemmArgs re{};
       re.slope = slope;
       re.A = a.e_in; re.K = a.Ke; re.R = csr.E; re.W = a.W_e; re.out = a.e_out;
+      re.wimg = tc_wimg(ctx, 1, layer); re.wfexp = tc_wfexp(ctx, 1, layer);
       re.pin = a.p; re.qin = a.q; re.src = csr.in_src; re.dst = csr.in_dst;
       if ((r = launch_rowgemm<D, EPI_EDGE>(ctx, re, "edge_tc", st)) < 0) return r;
       n += r;
@@ -1122,6 +1224,7 @@ static int tc_forward_layer_impl(const occu_ctx *ctx, const DevCsr &csr, const F
       RowGemmArgs rg{};
       rg.slope = slope;
       rg.A = a.e_out; rg.K = D; rg.R = csr.E; rg.W = a.W_m; rg.out = a.h_out;
+      rg.wimg = tc_wimg(ctx, 2, layer); rg.wfexp = tc_wfexp(ctx, 2, layer);
       rg.hbar = a.hbar; rg.src = csr.in_src; rg.dst = csr.in_dst; rg.in_ptr = csr.in_ptr;
       rg.mean = ctx->cfg.aggr == OCCU_AGGR_MEAN; rg.part = partial;
       if ((r = launch_rowgemm<D, EPI_GATEAGG>(ctx, rg, "gate_agg_tc", st)) < 0) return r;
@@ -1131,6 +1234,7 @@ static int tc_forward_layer_impl(const occu_ctx *ctx, const DevCsr &csr, const F
       RowGemmArgs rg{};
       rg.slope = slope;
       rg.A = a.e_out; rg.K = D; rg.R = csr.E; rg.W = a.W_m; rg.out = a.g;
+      rg.wimg = tc_wimg(ctx, 2, layer); rg.wfexp = tc_wfexp(ctx, 2, layer);
       if ((r = launch_rowgemm<D, EPI_GATE>(ctx, rg, "gate_tc", st)) < 0) return r;
       n += r;
     }
@@ -1155,64 +1259,67 @@ static int tc_forward_layer_impl(const occu_ctx *ctx, const DevCsr &csr, const F
 
 // ---- backward row-GEMMs on tensor cores ------------------------------------
 template <int D>
-static int bwd_gate_impl(const occu_ctx *ctx, const DevCsr &csr, const float *e, const float *W_m,
+static int bwd_gate_impl(const occu_ctx *ctx, const DevCsr &csr, int layer, const float *e,
                          const float *dh, const float *h, const float *hbar, float *MG, float *DV,
                          cudaStream_t st) {
   RowGemmArgs r{};
   r.slope = ctx->cfg.slope;
-  r.A = e; r.K = D; r.R = csr.E; r.W = W_m; r.out = MG; r.out2 = DV;
+  r.A = e; r.K = D; r.R = csr.E; r.out = MG; r.out2 = DV;
+  r.wimg = tc_wimg(ctx, 2, layer); r.wfexp = tc_wfexp(ctx, 2, layer);
   r.dh = dh; r.h = h; r.hbar = hbar; r.src = csr.in_src; r.dst = csr.in_dst;
   r.in_ptr = csr.in_ptr; r.mean = ctx->cfg.aggr == OCCU_AGGR_MEAN;
   return launch_rowgemm<D, EPI_GATEBWD>(ctx, r, "gate_bwd_tc", st);
 }
 template <int D>
-static int plain_impl(const occu_ctx *ctx, const float *A, int K, int R, const float *W, int transW,
+static int plain_impl(const occu_ctx *ctx, const float *A, int K, int R, int wkind, int layer,
                       const float *add, float *out, const char *name, cudaStream_t st,
                       const float *mask_h, const int32_t *in_ptr) {
   RowGemmArgs r{};
   r.slope = ctx->cfg.slope;
-  r.A = A; r.K = K; r.R = R; r.W = W; r.transW = transW; r.add = add; r.out = out;
+  r.A = A; r.K = K; r.R = R; r.add = add; r.out = out;
+  r.wimg = tc_wimg(ctx, wkind, layer); r.wfexp = tc_wfexp(ctx, wkind, layer);
   r.mask_h = mask_h; r.in_ptr = in_ptr; r.mean = ctx->cfg.aggr == OCCU_AGGR_MEAN;
   return launch_rowgemm<D, EPI_PLAIN>(ctx, r, name, st);
 }
 template <int D>
-static int bwd_edge_impl(const occu_ctx *ctx, const DevCsr &csr, const float *e_in, int Ke,
-                         const float *W_e, const float *e, const float *de, const float *p,
-                         const float *q, float *DZ, float *dal, cudaStream_t st) {
+static int bwd_edge_impl(const occu_ctx *ctx, const DevCsr &csr, int layer, const float *e_in,
+                         int Ke, const float *e, const float *de, const float *p, const float *q,
+                         float *DZ, float *dal, cudaStream_t st) {
   RowGemmArgs r{};
   r.slope = ctx->cfg.slope;
-  r.A = e_in; r.K = Ke; r.R = csr.E; r.W = W_e; r.out = DZ; r.dal = dal;
+  r.A = e_in; r.K = Ke; r.R = csr.E; r.out = DZ; r.dal = dal;
+  r.wimg = tc_wimg(ctx, 1, layer); r.wfexp = tc_wfexp(ctx, 1, layer);
   r.e = e; r.de = de; r.pin = p; r.qin = q; r.src = csr.in_src; r.dst = csr.in_dst;
   return launch_rowgemm<D, EPI_EDGEBWD>(ctx, r, "edge_bwd_tc", st);
 }
 
-int launch_bwd_gate_tc(const occu_ctx *ctx, const DevCsr &csr, const float *e, const float *W_m,
+int launch_bwd_gate_tc(const occu_ctx *ctx, const DevCsr &csr, int layer, const float *e,
                        const float *dh, const float *h, const float *hbar, float *MG, float *DV,
                        cudaStream_t st) {
   if (csr.E <= 0) return 0;
-  return ctx->cfg.d == 64 ? bwd_gate_impl<64>(ctx, csr, e, W_m, dh, h, hbar, MG, DV, st)
-                          : bwd_gate_impl<128>(ctx, csr, e, W_m, dh, h, hbar, MG, DV, st);
+  return ctx->cfg.d == 64 ? bwd_gate_impl<64>(ctx, csr, layer, e, dh, h, hbar, MG, DV, st)
+                          : bwd_gate_impl<128>(ctx, csr, layer, e, dh, h, hbar, MG, DV, st);
 }
-int launch_plain_tc(const occu_ctx *ctx, const float *A, int K, int R, const float *W, int transW,
+int launch_plain_tc(const occu_ctx *ctx, const float *A, int K, int R, int wkind, int layer,
                     const float *add, float *out, const char *name, cudaStream_t st,
                     const float *mask_h, const int32_t *in_ptr) {
   if (R <= 0) return 0;
-  return ctx->cfg.d == 64 ? plain_impl<64>(ctx, A, K, R, W, transW, add, out, name, st, mask_h, in_ptr)
-                          : plain_impl<128>(ctx, A, K, R, W, transW, add, out, name, st, mask_h, in_ptr);
+  return ctx->cfg.d == 64 ? plain_impl<64>(ctx, A, K, R, wkind, layer, add, out, name, st, mask_h, in_ptr)
+                          : plain_impl<128>(ctx, A, K, R, wkind, layer, add, out, name, st, mask_h, in_ptr);
 }
-int launch_bwd_edge_tc(const occu_ctx *ctx, const DevCsr &csr, const float *e_in, int Ke,
-                       const float *W_e, const float *e, const float *de, const float *p,
-                       const float *q, float *DZ, float *dal, cudaStream_t st) {
+int launch_bwd_edge_tc(const occu_ctx *ctx, const DevCsr &csr, int layer, const float *e_in, int Ke,
+                       const float *e, const float *de, const float *p, const float *q, float *DZ,
+                       float *dal, cudaStream_t st) {
   if (csr.E <= 0) return 0;
-  return ctx->cfg.d == 64 ? bwd_edge_impl<64>(ctx, csr, e_in, Ke, W_e, e, de, p, q, DZ, dal, st)
-                          : bwd_edge_impl<128>(ctx, csr, e_in, Ke, W_e, e, de, p, q, DZ, dal, st);
+  return ctx->cfg.d == 64 ? bwd_edge_impl<64>(ctx, csr, layer, e_in, Ke, e, de, p, q, DZ, dal, st)
+                          : bwd_edge_impl<128>(ctx, csr, layer, e_in, Ke, e, de, p, q, DZ, dal, st);
 }
 
-int launch_forward_layer_tc(const occu_ctx *ctx, const DevCsr &csr, const FwdLayerArgs &a,
+int launch_forward_layer_tc(const occu_ctx *ctx, const DevCsr &csr, int layer, const FwdLayerArgs &a,
                             float *partial, cudaStream_t st) {
   switch (ctx->cfg.d) {
-    case 64: return tc_forward_layer_impl<64>(ctx, csr, a, partial, st);
-    case 128: return tc_forward_layer_impl<128>(ctx, csr, a, partial, st);
+    case 64: return tc_forward_layer_impl<64>(ctx, csr, layer, a, partial, st);
+    case 128: return tc_forward_layer_impl<128>(ctx, csr, layer, a, partial, st);
     default: return -int(cudaErrorInvalidValue);
   }
 }

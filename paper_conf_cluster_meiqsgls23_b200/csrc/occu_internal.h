@@ -87,7 +87,9 @@ struct occu_ctx {
   int num_sms = 148;
   bool weights_ready = false;
   bool keep = false;
-  int path = 0;            // 0: tensor cores (3xTF32), 1: CUDA-core SIMT FP32
+  int path = 0;            // 0: tensor cores, 1: CUDA-core SIMT FP32, 2: tensor cores + fused aggregation
+  occu::DevBuf wimg, wjobs, wfexp;   // prebuilt tensor-core weight images (per parameter version)
+  int64_t params_version = 0, wimg_version = -1;
   float weight_decay = 1e-4f;
   occu::DevBuf params, grads, adam_m, adam_v;
   int64_t adam_t = 0;
@@ -119,20 +121,24 @@ struct FwdLayerArgs {
 int launch_forward_layer(const occu_ctx *ctx, const DevCsr &csr, const FwdLayerArgs &a,
                          cudaStream_t st);
 bool tc_supported(const occu_config &c);
+// Weight images for the tensor-core row-GEMMs; kind: 0 W_u, 1 W_e, 2 W_m, 3 W_mᵀ, 4 W_eᵀ, 5 W_uᵀ.
+int tc_prepare_weights(occu_ctx *ctx, cudaStream_t st);
+const uint8_t *tc_wimg(const occu_ctx *ctx, int kind, int layer);
+const int *tc_wfexp(const occu_ctx *ctx, int kind, int layer);
 bool wgrad_tc_supported(int A, int Bn);
-int launch_bwd_gate_tc(const occu_ctx *ctx, const DevCsr &csr, const float *e, const float *W_m,
+int launch_bwd_gate_tc(const occu_ctx *ctx, const DevCsr &csr, int layer, const float *e,
                        const float *dh, const float *h, const float *hbar, float *MG, float *DV,
                        cudaStream_t st);
-int launch_plain_tc(const occu_ctx *ctx, const float *A, int K, int R, const float *W, int transW,
+int launch_plain_tc(const occu_ctx *ctx, const float *A, int K, int R, int wkind, int layer,
                     const float *add, float *out, const char *name, cudaStream_t st,
                     const float *mask_h = nullptr, const int32_t *in_ptr = nullptr);
-int launch_bwd_edge_tc(const occu_ctx *ctx, const DevCsr &csr, const float *e_in, int Ke,
-                       const float *W_e, const float *e, const float *de, const float *p,
+int launch_bwd_edge_tc(const occu_ctx *ctx, const DevCsr &csr, int layer, const float *e_in, int Ke,
+                       const float *e, const float *de, const float *p,
                        const float *q, float *DZ, float *dal, cudaStream_t st);
 int launch_wgrad_tc(const occu_ctx *ctx, const float *X, int A, const float *Y, int Bn, long R,
                     int splits, float *partial, cudaStream_t st);
 size_t tc_partial_floats(int E, int D);
-int launch_forward_layer_tc(const occu_ctx *ctx, const DevCsr &csr, const FwdLayerArgs &a,
+int launch_forward_layer_tc(const occu_ctx *ctx, const DevCsr &csr, int layer, const FwdLayerArgs &a,
                             float *partial, cudaStream_t st);
 int launch_gather_segsum(const occu_ctx *ctx, const DevCsr &csr, const float *g,
                          const float *hbar, float *h_out, cudaStream_t st);

@@ -225,6 +225,7 @@ occu_status forward(occu_ctx *ctx, const DevCsr &csr, const float *nf, const flo
   cudaStream_t s = ctx->stream;
   const float *P = ctx->params.as<float>();
   LK(launch_permute_rows(ctx, ef, csr.in_eid, csr.E, c.F_e, w.e0.as<float>(), s), "permute e0");
+  if (ctx->path != 1 && tc_supported(c)) LK(tc_prepare_weights(ctx, s), "weight images");
   for (int i = 0; i < c.L; ++i) {
     FwdLayerArgs a{};
     a.h_in = i == 0 ? nf : w.h[i - 1].as<float>();
@@ -240,7 +241,7 @@ occu_status forward(occu_ctx *ctx, const DevCsr &csr, const float *nf, const flo
     if (ctx->path != 1 && tc_supported(c)) {
       a.e_out = w.e[i].as<float>();            // the gate kernel re-reads e'
       CK(w.tcpart.ensure(tc_partial_floats(csr.E, c.d) * 4), "alloc tc partials");
-      LK(launch_forward_layer_tc(ctx, csr, a, w.tcpart.as<float>(), s), "forward layer (tc)");
+      LK(launch_forward_layer_tc(ctx, csr, i, a, w.tcpart.as<float>(), s), "forward layer (tc)");
     } else {
       LK(launch_forward_layer(ctx, csr, a, s), "forward layer");
     }
@@ -389,6 +390,9 @@ occu_status occu_destroy(occu_ctx *ctx) {
   if (ctx->comm) ncclCommDestroy(ctx->comm);
   ctx->ws.release_all();
   ctx->params.release();
+  ctx->wimg.release();
+  ctx->wjobs.release();
+  ctx->wfexp.release();
   ctx->grads.release();
   ctx->adam_m.release();
   ctx->adam_v.release();
@@ -409,6 +413,7 @@ occu_status occu_set_params(occu_ctx *ctx, const float *host_flat, size_t n) {
   CK(cudaMemcpyAsync(ctx->params.ptr, host_flat, n * 4, cudaMemcpyHostToDevice, ctx->stream), "H2D");
   CK(cudaStreamSynchronize(ctx->stream), "sync");
   ctx->weights_ready = true;
+  ctx->params_version += 1;
   return OCCU_OK;
 }
 

@@ -27,7 +27,7 @@ m.predict(csr, nf, ef); torch.cuda.synchronize()
 L.occu_debug_tc_time(buf.ctypes.data_as(ctypes.c_void_p))   # reset
 m.predict(csr, nf, ef); torch.cuda.synchronize()
 L.occu_debug_tc_time(buf.ctypes.data_as(ctypes.c_void_p))
-names = ["producer", "mma"] + [f"conv{w}" for w in range(4)] + [f"epi{w}" for w in range(16)]
+names = ["producer", "mma"] + [f"conv{w}" for w in range(8)] + [f"epi{w}" for w in range(16)] + ["-", "-", "-", "-", "setup", "total"]
 for k, n in enumerate(names):
     w, bsy, cnt = buf[k][0], buf[k][1], buf[k][2]
     if cnt:
