@@ -13,6 +13,8 @@
 #include "nccl.h"
 #include "occu_internal.h"
 
+void occu_host_batch_release(occu_csr_batch *b);
+
 namespace occu {
 void init_flat(const occu_config &c, uint64_t seed, std::vector<float> &out);
 bool write_file(const char *path, const char magic[8], const occu_config &c,
@@ -496,9 +498,12 @@ occu_status occu_batch_to_device(occu_ctx *ctx, const occu_csr_batch *host, occu
 
 void occu_batch_free(occu_csr_batch *b) {
   if (!b) return;
-  if (b->on_device) cudaFree(b->priv);
-  else free(b->priv);
-  free(b);
+  if (b->on_device) {
+    cudaFree(b->priv);
+    free(b);
+  } else {
+    occu_host_batch_release(b);
+  }
 }
 
 occu_status occu_predict(occu_ctx *ctx, const occu_csr_batch *csr_batch, const float *node_feat,

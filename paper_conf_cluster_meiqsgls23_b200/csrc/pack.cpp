@@ -13,12 +13,114 @@
 
 #include <algorithm>
 #include <atomic>
+#include <condition_variable>
+#include <functional>
+#include <mutex>
 #include <thread>
 #include <vector>
 
 #include "occu_internal.h"
 
 namespace {
+
+// Small pool of host output buffers: repeated packing of same-sized batches reuses
+// already-faulted memory instead of paying mmap/page-fault costs on every call.
+std::mutex g_pool_mu;
+std::vector<std::pair<void *, size_t>> g_pool;
+
+void *pool_take(size_t bytes, size_t *cap) {
+  std::lock_guard<std::mutex> lk(g_pool_mu);
+  for (size_t i = 0; i < g_pool.size(); ++i)
+    if (g_pool[i].second >= bytes && g_pool[i].second <= 2 * bytes + 4096) {
+      void *p = g_pool[i].first;
+      *cap = g_pool[i].second;
+      g_pool.erase(g_pool.begin() + i);
+      return p;
+    }
+  *cap = bytes;
+  return malloc(bytes);
+}
+
+// Persistent worker pool for per-graph packing (no thread creation per call).
+class PackPool {
+ public:
+  explicit PackPool(int n) {
+    for (int t = 0; t < n; ++t) workers_.emplace_back([this] { loop(); });
+  }
+  ~PackPool() {
+    {
+      std::lock_guard<std::mutex> lk(mu_);
+      stop_ = true;
+    }
+    cv_.notify_all();
+    for (auto &w : workers_) w.join();
+  }
+  int size() const { return int(workers_.size()); }
+  // Runs fn(i) for i in [0, n) on the pool plus the calling thread; returns when done.
+  template <class F> void run(int n, F fn) {
+    std::function<void(int)> f = fn;
+    {
+      std::lock_guard<std::mutex> lk(mu_);
+      job_ = &f;
+      n_ = n;
+      next_ = 0;
+      active_ = int(workers_.size());
+      ++gen_;
+    }
+    cv_.notify_all();
+    for (;;) {
+      const int i = next_.fetch_add(1);
+      if (i >= n) break;
+      f(i);
+    }
+    std::unique_lock<std::mutex> lk(mu_);
+    done_cv_.wait(lk, [this] { return active_ == 0; });
+    job_ = nullptr;
+  }
+
+ private:
+  void loop() {
+    uint64_t seen = 0;
+    for (;;) {
+      std::function<void(int)> *job;
+      int n;
+      {
+        std::unique_lock<std::mutex> lk(mu_);
+        cv_.wait(lk, [&] { return stop_ || gen_ != seen; });
+        if (stop_) return;
+        seen = gen_;
+        job = job_;
+        n = n_;
+      }
+      for (;;) {
+        const int i = next_.fetch_add(1);
+        if (i >= n) break;
+        (*job)(i);
+      }
+      std::lock_guard<std::mutex> lk(mu_);
+      if (--active_ == 0) done_cv_.notify_all();
+    }
+  }
+  std::vector<std::thread> workers_;
+  std::mutex mu_;
+  std::condition_variable cv_, done_cv_;
+  std::function<void(int)> *job_ = nullptr;
+  int n_ = 0, active_ = 0;
+  std::atomic<int> next_{0};
+  uint64_t gen_ = 0;
+  bool stop_ = false;
+};
+
+PackPool &pack_pool() {
+  static PackPool pool([] {
+    unsigned hw = std::thread::hardware_concurrency();
+    const char *env = getenv("OCCU_PACK_THREADS");
+    if (env) hw = unsigned(atoi(env));
+    if (hw < 1) hw = 1;
+    return int(std::min(hw, 32u)) - 1;
+  }());
+  return pool;
+}
 
 struct Scratch {
   std::vector<int32_t> cnt, tmp;
@@ -116,7 +218,8 @@ extern "C" occu_status occu_pack(const occu_graph_view *graphs, int32_t num_grap
   // one allocation for all arrays
   const size_t B1 = num_graphs + 1, N1 = N + 1;
   const size_t total = 2 * B1 + 2 * N1 + 4 * static_cast<size_t>(E) + static_cast<size_t>(N);
-  int32_t *base = static_cast<int32_t *>(malloc(std::max<size_t>(total, 1) * sizeof(int32_t)));
+  size_t cap = 0;
+  int32_t *base = static_cast<int32_t *>(pool_take(std::max<size_t>(total, 1) * sizeof(int32_t), &cap));
   if (!base) {
     free(b);
     return OCCU_ENOMEM;
@@ -141,29 +244,27 @@ extern "C" occu_status occu_pack(const occu_graph_view *graphs, int32_t num_grap
   }
   b->in_ptr[N] = static_cast<int32_t>(E);
   b->out_ptr[N] = static_cast<int32_t>(E);
-  // parallel over graphs (work-stealing by atomic counter; results independent of order)
-  unsigned hw = std::thread::hardware_concurrency();
-  const char *env = getenv("OCCU_PACK_THREADS");
-  if (env) hw = static_cast<unsigned>(atoi(env));
-  int nthreads = static_cast<int>(std::min<int64_t>(std::max(1u, hw), num_graphs));
-  if (E + N < 20000) nthreads = 1;
-  std::atomic<int32_t> next{0};
-  auto worker = [&]() {
-    Scratch s;
-    for (;;) {
-      const int32_t i = next.fetch_add(1);
-      if (i >= num_graphs) break;
-      pack_graph(graphs[i], b->node_off[i], b->edge_off[i], b, s);
-      for (int32_t v = b->node_off[i]; v < b->node_off[i + 1]; ++v) b->node_graph[v] = i;
-    }
+  // parallel over graphs on a persistent pool (results independent of schedule)
+  auto one = [&](int i) {
+    thread_local Scratch s;
+    pack_graph(graphs[i], b->node_off[i], b->edge_off[i], b, s);
+    for (int32_t v = b->node_off[i]; v < b->node_off[i + 1]; ++v) b->node_graph[v] = i;
   };
-  if (nthreads <= 1) {
-    worker();
+  if (E + N < 20000 || pack_pool().size() == 0) {
+    for (int32_t i = 0; i < num_graphs; ++i) one(i);
   } else {
-    std::vector<std::thread> pool;
-    for (int t = 0; t < nthreads; ++t) pool.emplace_back(worker);
-    for (auto &t : pool) t.join();
+    pack_pool().run(num_graphs, one);
   }
   *out = b;
   return OCCU_OK;
+}
+
+// Host batches return their buffer to the pool (runtime frees device batches).
+void occu_host_batch_release(occu_csr_batch *b) {
+  std::lock_guard<std::mutex> lk(g_pool_mu);
+  const size_t total = 2 * size_t(b->num_graphs + 1) + 2 * size_t(b->num_nodes + 1) +
+                       4 * size_t(b->num_edges) + size_t(b->num_nodes);
+  if (g_pool.size() < 4) g_pool.push_back({b->priv, std::max<size_t>(total, 1) * sizeof(int32_t)});
+  else free(b->priv);
+  free(b);
 }

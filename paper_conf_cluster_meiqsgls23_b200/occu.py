@@ -191,22 +191,36 @@ class Csr:
             self._p = None
 
 
+_VIEW_DT = np.dtype([("num_nodes", "<i4"), ("num_edges", "<i4"), ("src", "<u8"), ("dst", "<u8")],
+                    align=True)
+
+
 def pack(graphs) -> Csr:
-    """graphs: list of (num_nodes, src int32[m], dst int32[m]) with local ids."""
+    """graphs: list of (num_nodes, src int32[m], dst int32[m]) with local ids.
+
+    Builds the occu_graph_view array with NumPy (one concatenation, pointer
+    arithmetic) and calls occu_pack; packing itself runs in the library."""
     n = len(graphs)
-    views = (GraphView * max(n, 1))()
-    keep = []
-    for i, (nn, s, t) in enumerate(graphs):
-        s = np.ascontiguousarray(s, dtype=np.int32)
-        t = np.ascontiguousarray(t, dtype=np.int32)
-        keep += [s, t]
-        views[i].num_nodes = int(nn)
-        views[i].num_edges = int(len(s))
-        views[i].src = s.ctypes.data_as(C.POINTER(C.c_int32))
-        views[i].dst = t.ctypes.data_as(C.POINTER(C.c_int32))
+    assert ctypes_view_ok()
+    nn = np.fromiter((g[0] for g in graphs), dtype=np.int32, count=n)
+    m = np.fromiter((len(g[1]) for g in graphs), dtype=np.int64, count=n)
+    src = np.concatenate([np.asarray(g[1], dtype=np.int32) for g in graphs]) if n else np.zeros(0, np.int32)
+    dst = np.concatenate([np.asarray(g[2], dtype=np.int32) for g in graphs]) if n else np.zeros(0, np.int32)
+    src = np.ascontiguousarray(src)
+    dst = np.ascontiguousarray(dst)
+    off = np.concatenate([[0], np.cumsum(m)[:-1]]).astype(np.uint64) * np.uint64(4)
+    views = np.zeros(max(n, 1), dtype=_VIEW_DT)
+    views["num_nodes"][:n] = nn
+    views["num_edges"][:n] = m.astype(np.int32)
+    views["src"][:n] = np.uint64(src.ctypes.data) + off
+    views["dst"][:n] = np.uint64(dst.ctypes.data) + off
     out = C.POINTER(CsrBatch)()
-    _check(lib().occu_pack(views, n, C.byref(out)))
+    _check(lib().occu_pack(views.ctypes.data_as(C.POINTER(GraphView)), n, C.byref(out)))
     return Csr(out)
+
+
+def ctypes_view_ok() -> bool:
+    return _VIEW_DT.itemsize == C.sizeof(GraphView)
 
 
 class Model:
