@@ -8,8 +8,11 @@ os.makedirs(out, exist_ok=True)
 def kname(full):
     m = re.search(r"rowgemm_kernel<(\d+), (\d+)>", full)
     if m:
-        return ["node_tc", "edge_tc", "gate_tc"][int(m.group(2))]
-    for k, v in [("edge_small", "edge_small"), ("gather_segsum", "gather_segsum"),
+        return ["node_tc", "edge_tc", "gate_tc", "plain_tc", "gatebwd_tc", "edgebwd_tc",
+                "gateagg_tc"][int(m.group(2))]
+    for k, v in [("edge_small", "edge_small"), ("wgrad_tc", "wgrad_tc"), ("wimage", "wimage"),
+                 ("split_reduce", "split_reduce"), ("agg_fixup", "agg_fixup"),
+                 ("wgrad_skinny", "wgrad_skinny"), ("gather_segsum", "gather_segsum"),
                  ("readout_head", "readout_head"), ("permute_rows", "permute_e0"),
                  ("node_gemm_kernel", "node_gemm"), ("edge_fwd_kernel", "edge_fwd"),
                  ("edge_bwd_m", "edge_bwd_m"), ("edge_bwd_e", "edge_bwd_e"), ("node_bwd", "node_bwd"),
@@ -49,40 +52,50 @@ if os.path.exists(lp):
         print(f"  {k:16s} {a[0]:4d} {100*a[1]/tot:6.1f}% {a[2]/a[0]/1e6:9.1f} MB")
 
 # 2) full capture -> traffic per launch for the hot kernels
-fp = os.path.join(ROOT, "gpurun_out", "prof_full.ncu-rep")
 traffic = {}
 lines = []
-if os.path.exists(fp):
-    raw = subprocess.run(["ncu", "-i", fp, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
-    rows = list(csv.reader(io.StringIO(raw)))
-    hdr = rows[0]
-    def g(r, k):
-        try:
-            return float(r[hdr.index(k)].replace(",", ""))
-        except Exception:
-            return None
-    acc = collections.defaultdict(list)
-    for r in rows[2:]:
-        k = kname(r[hdr.index("Kernel Name")])
-        unit_r = rows[1][hdr.index("dram__bytes_read.sum")]
-        scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9}.get(unit_r, 1)
-        acc[k].append({
-            "time_us": g(r, "gpu__time_duration.sum"),
-            "dram_bytes": (g(r, "dram__bytes_read.sum") + g(r, "dram__bytes_write.sum")) * scale,
-            "dram_pct": g(r, "dram__throughput.avg.pct_of_peak_sustained_elapsed"),
-            "tensor_pct": g(r, "sm__pipe_tensor_cycles_active.avg.pct_of_peak_sustained_elapsed"),
-            "issue_pct": g(r, "smsp__issue_active.avg.pct_of_peak_sustained_active"),
-            "regs": g(r, "launch__registers_per_thread"),
-        })
-    for k, lst in acc.items():
-        n = len(lst)
-        traffic[k] = {"dram_bytes_per_launch": sum(x["dram_bytes"] for x in lst) / n,
-                      "launches_captured": n,
-                      "mean_time_us_under_ncu": sum(x["time_us"] or 0 for x in lst) / n,
-                      "dram_throughput_pct": sum(x["dram_pct"] or 0 for x in lst) / n,
-                      "tensor_pipe_pct": sum(x["tensor_pct"] or 0 for x in lst) / n,
-                      "issue_active_pct": sum(x["issue_pct"] or 0 for x in lst) / n,
-                      "registers": lst[0]["regs"],
-                      "source": f"profiles/{tag}: ncu --set full, scripts/prof_driver.py (CFG2)"}
-    json.dump(traffic, open(os.path.join(out, "traffic.json"), "w"), indent=1)
-    print(json.dumps(traffic, indent=1))
+for rep, drv in (("prof_full", "scripts/prof_driver.py (CFG2 inference)"),
+                 ("prof_train", "scripts/prof_driver.py --train (CFG2 training)")):
+  fp = os.path.join(ROOT, "gpurun_out", rep + ".ncu-rep")
+  if os.path.exists(fp):
+      raw = subprocess.run(["ncu", "-i", fp, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
+      rows = list(csv.reader(io.StringIO(raw)))
+      hdr = rows[0]
+      def g(r, k):
+          try:
+              return float(r[hdr.index(k)].replace(",", ""))
+          except Exception:
+              return None
+      acc = collections.defaultdict(list)
+      for r in rows[2:]:
+          k = kname(r[hdr.index("Kernel Name")])
+          unit_r = rows[1][hdr.index("dram__bytes_read.sum")]
+          scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9}.get(unit_r, 1)
+          acc[k].append({
+              "time_us": g(r, "gpu__time_duration.sum"),
+              "dram_bytes": (g(r, "dram__bytes_read.sum") + g(r, "dram__bytes_write.sum")) * scale,
+              "dram_pct": g(r, "gpu__dram_throughput.avg.pct_of_peak_sustained_elapsed"),
+              "tensor_pct": g(r, "sm__pipe_tensor_cycles_active.avg.pct_of_peak_sustained_elapsed"),
+              "issue_pct": g(r, "smsp__issue_active.avg.pct_of_peak_sustained_active"),
+              "regs": g(r, "launch__registers_per_thread"),
+          })
+      for k, lst in acc.items():
+          n = len(lst)
+          traffic[k] = {"dram_bytes_per_launch": sum(x["dram_bytes"] for x in lst) / n,
+                        "launches_captured": n,
+                        "mean_time_us_under_ncu": sum(x["time_us"] or 0 for x in lst) / n,
+                        "dram_throughput_pct": sum(x["dram_pct"] or 0 for x in lst) / n,
+                        "tensor_pipe_pct": sum(x["tensor_pct"] or 0 for x in lst) / n,
+                        "issue_active_pct": sum(x["issue_pct"] or 0 for x in lst) / n,
+                        "registers": lst[0]["regs"],
+                        "source": f"profiles/{tag}: ncu --set full, {drv}"}
+json.dump(traffic, open(os.path.join(out, "traffic.json"), "w"), indent=1)
+with open(os.path.join(out, f"{tag}_ncu_summary.md"), "w") as f:
+    f.write(f"# {tag}: ncu --set full --clock-control none (serialised, cold-cache replays)\n\n")
+    f.write("| kernel | launches | us/launch (ncu) | DRAM MB/launch | DRAM % peak | tensor pipe % | issue active % | regs |\n")
+    f.write("|---|---|---|---|---|---|---|---|\n")
+    for k, t in traffic.items():
+        f.write(f"| {k} | {t['launches_captured']} | {t['mean_time_us_under_ncu']:.1f} | "
+                f"{t['dram_bytes_per_launch']/1e6:.1f} | {t['dram_throughput_pct']:.1f} | "
+                f"{t['tensor_pipe_pct']:.1f} | {t['issue_active_pct']:.1f} | {t['registers']:.0f} |\n")
+print(open(os.path.join(out, f"{tag}_ncu_summary.md")).read())
