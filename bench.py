@@ -107,25 +107,37 @@ def dist_env():
 # ---------------------------------------------------------------- algorithmic bytes
 # Bytes each kernel must move per step (all its launches), fp32 storage, d = 128,
 # with perfect reuse of gathered rows (each h̄ / p / q row counted once).  DESIGN.md §6.
-def algorithmic_bytes(N, E, B, d=128, F_n=80, F_e=4, L=3):
+def readout_rows(graphs, chunk=8):
+    """Rows of readout chunk partials the fused last aggregation writes: one per
+    (graph, 8-node chunk) pair the graph touches."""
+    off = np.concatenate([[0], np.cumsum([int(n) for n, _, _ in graphs])])
+    return int(np.sum((off[1:] - 1) // chunk - off[:-1] // chunk + 1))
+
+
+def algorithmic_bytes(N, E, B, d=128, F_n=80, F_e=4, L=3, rrows=None):
+    """Per-step algorithmic bytes per kernel class (fp32 values, int32 indices).
+    rrows: readout partial rows when the readout is folded into the last aggregation
+    and the layer-1 edge kernel gathers edge_feat through in_eid (kernel path 0)."""
     s = 4
+    fused = rrows is not None
     node = s * N * F_n + s * N * d * (L - 1) + s * N * (d + 2) * L                # read h_in, write h̄,p,q
-    edge_small = s * E * F_e + 8 * E + 8 * N + s * E * d                          # layer 1
+    edge_small = s * E * F_e + 8 * E + 8 * N + s * E * d + (4 * E if fused else 0)  # layer 1
     edge_tc = (L - 1) * (s * E * d + 8 * E + 8 * N + s * E * d)                    # layers 2..L
     gate = L * (s * E * d + s * E * d)                                             # read e', write g
-    gather = L * (s * E * d + s * N * d + 4 * E + 4 * (N + 1) + s * N * d)         # g, h̄, idx, h
-    readout = s * N * d + s * B * (2 * d + 1)
-    permute = s * E * F_e * 2 + 4 * E
-    return {"node_tc": node, "edge_small": edge_small, "edge_tc": edge_tc, "gate_tc": gate,
-            "gather_segsum": gather, "readout_head": readout, "permute_e0": permute,
-            # SIMT path kernels
-            "node_gemm": node, "edge_fwd": edge_small + edge_tc + gate}
-
-
-def aggregation_bytes(N, E, d, s=4):
-    """a5 + a6 per launch (gather_segsum): read g [E,d], gather h̄[src] once per node,
-    read in_src / in_ptr, write h [N,d]."""
-    return s * (E * d + N * d + N * d) + 4 * (E + N + 1)
+    gather = L * (s * E * d + s * N * d + 4 * E + 4 * (N + 1))                     # g, h̄, idx
+    if fused:
+        gather += (L - 1) * s * N * d + 4 * N + s * rrows * d                      # h, node_graph, partials
+        readout = s * rrows * d + 4 * (B + 1) + s * B * (2 * d + 1)
+    else:
+        gather += L * s * N * d
+        readout = s * N * d + s * B * (2 * d + 1)
+    out = {"node_tc": node, "edge_small": edge_small, "edge_tc": edge_tc, "gate_tc": gate,
+           "gather_segsum": gather, "readout_head": readout,
+           # SIMT path kernels
+           "node_gemm": node, "edge_fwd": edge_small + edge_tc + gate}
+    if not fused:
+        out["permute_e0"] = s * E * F_e * 2 + 4 * E
+    return out
 
 
 def load_traffic():
@@ -297,7 +309,11 @@ def main():
     with ClockSampler(local) as clk:
         timed(infer, args.warmup)
         bar()
-        times, launches = timed(infer, args.steps, profile=True)
+        times, launches = timed(infer, args.steps)
+        bar()
+        # per-kernel CUDA events (library profiler) over a second timed pass of the
+        # same K steps: the headline above carries no event records between kernels
+        ptimes, _ = timed(infer, args.steps, profile=True)
         bar()
         t_end = time.time() + 0.5
         while time.time() < t_end:
@@ -306,12 +322,13 @@ def main():
             torch.cuda.synchronize()
     prof = model.profile()
     ms_step = max_over_ranks(float(np.sum(times)) / args.steps)
+    ms_step_prof = max_over_ranks(float(np.sum(ptimes)) / args.steps)
     value = B * world / (ms_step * 1e-3)
 
     # roofline: per-kernel device time inside the timed region (CUDA events on the
     # library's launch stream), algorithmic bytes per kernel
     d = 128
-    alg = algorithmic_bytes(N, E, B, d)
+    alg = algorithmic_bytes(N, E, B, d, rrows=readout_rows(batch.graphs) if args.path == 0 else None)
     traffic = load_traffic()
     kernels = {}
     for k, (ms_tot, n) in prof.items():
@@ -334,7 +351,7 @@ def main():
             "share_of_step": kd["ms_per_step"] / tot_kernel if tot_kernel else None}
     agg_ms = kernels.get("gather_segsum", {}).get("ms_per_step")
     agg_launch = agg_ms / 3 if agg_ms else None
-    agg_b = aggregation_bytes(N, E, d)
+    agg_b = alg["gather_segsum"] / 3          # mean per launch over the L = 3 layers
     agg = {"kernel": "gather_segsum", "bound": "hbm", "algorithmic_bytes_per_launch": agg_b,
            "avg_ms": agg_launch,
            "achieved": agg_b / (agg_launch * 1e-3) / 1e9 if agg_launch else None,
@@ -403,7 +420,7 @@ def main():
             "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
             "config": {"workload": "CFG2 (BASELINE.json configs[1])", "graphs_per_rank": B,
                        "nodes_per_rank": N, "edges_per_rank": E, "L": 3, "d": 128, "F_n": 80,
-                       "F_e": 4, "precision": "fp32: tcgen05 3xTF32 split GEMMs, FP32 accumulate" if args.path == 0 else "fp32 (SIMT)",
+                       "F_e": 4, "precision": "fp32: tcgen05 fp16x2-split GEMMs (3 products), FP32 accumulate" if args.path != 1 else "fp32 (SIMT)",
                        "l2": "flushed between timed steps (256 MiB write)" if not args.no_flush else "not flushed",
                        "parallelism": f"graph-sharded x{world}, no collective"},
             "gpu_launches": launches,
@@ -412,6 +429,9 @@ def main():
             "aggregation": agg,
             "kernel_ms_per_step": {k: v["ms_per_step"] for k, v in kernels.items()},
             "kernels": kernels,
+            "kernel_timing": {"how": "CUDA events around every library launch (on its stream) "
+                                     "over a second timed pass of the same K steps",
+                              "ms_per_step_with_events": ms_step_prof},
             "e2e": e2e,
             "train": train,
             "cpu_baseline": cpu,

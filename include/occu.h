@@ -175,7 +175,10 @@ typedef enum {
  * into one tensor-core kernel; 1 = CUDA-core FP32 (SIMT) everywhere.  All meet
  * the FP32 tolerance. */
 occu_status occu_set_kernel_path(occu_ctx *ctx, int path);
-/* Keep every intermediate of the next forward (costs memory/bandwidth). */
+/* Keep every intermediate of the next forward (costs memory/bandwidth).  Without
+ * it, the last layer's e and (kernel path 0) h are not stored: path 0 folds the
+ * readout's node sums into the last aggregation, and occu_get_tensor returns
+ * OCCU_ENOTREADY for them. */
 occu_status occu_set_keep_intermediates(occu_ctx *ctx, int keep);
 /* Copy an intermediate of the last forward into host memory (float32; BF16
  * precision stores are widened).  bytes must equal the tensor size. */

@@ -271,19 +271,34 @@ __global__ void __launch_bounds__(NT) edge_fwd_kernel(
   }
 }
 
+template <int V>
+__device__ __forceinline__ void store_row(float *dst, const float (&v)[V]) {
+  if constexpr (V == 4) {
+    *reinterpret_cast<float4 *>(dst) = make_float4(v[0], v[1], v[2], v[3]);
+  } else {
+#pragma unroll
+    for (int c = 0; c < V; ++c) dst[c] = v[c];
+  }
+}
+
 // ---------------------------------------------------------------------------
 // a5 + a6: gather + deterministic segmented sum, warp per destination node.
 // Lane l owns channels [l*V, l*V+V), V = D/32; edges summed in ascending k.
 // ---------------------------------------------------------------------------
-template <int D>
+template <int D, bool RP>
 __global__ void __launch_bounds__(NT) gather_segsum_kernel(
     const float *__restrict__ g, const float *__restrict__ hbar,
     const int32_t *__restrict__ in_ptr, const int32_t *__restrict__ in_src, int N, int mean,
-    float slope, float *__restrict__ h_out) {
-  // A warp owns NPW consecutive destination nodes, i.e. the contiguous in-CSR edge
-  // range [in_ptr[t0], in_ptr[t0+NPW]); edges are consumed in ascending order, four
-  // gathered rows in flight at a time, and each node's sum is flushed when the edge
-  // index crosses its segment end (fixed order: identical to a per-node loop).
+    float slope, float *__restrict__ h_out, const int32_t *__restrict__ node_graph,
+    float *__restrict__ rpart) {
+  // A warp owns NPW consecutive destination nodes (a "chunk"), i.e. the contiguous
+  // in-CSR edge range [in_ptr[t0], in_ptr[t0+NPW]); edges are consumed in ascending
+  // order, four gathered rows in flight at a time, and each node's sum is flushed when
+  // the edge index crosses its segment end (fixed order: identical to a per-node loop).
+  // Last layer (rpart != null): the flushed rows h_u are also summed per graph inside
+  // the chunk, in ascending u, and graph b's chunk partial is stored at row
+  // min(u1 - 1, t0 + NPW - 1) of rpart (its last node in the chunk) for
+  // readout_head_kernel (a7); h_out may then be null (inference never re-reads h_L).
   constexpr int V = D / 32;
   constexpr int NPW = 8;
   const int lane = threadIdx.x & 31;
@@ -291,22 +306,41 @@ __global__ void __launch_bounds__(NT) gather_segsum_kernel(
   for (long t0 = (blockIdx.x * long(NT) + threadIdx.x) / 32 * NPW; t0 < N; t0 += warps * NPW) {
     const int nn = int(min(long(NPW), N - t0));
     const int ptr_l = lane <= nn ? in_ptr[t0 + lane] : 0;      // in_ptr[t0 .. t0+nn]
+    const int gr_l = (RP && lane < nn) ? node_graph[t0 + lane] : -1;
     const int e_beg = __shfl_sync(0xffffffffu, ptr_l, 0);
     const int e_end = __shfl_sync(0xffffffffu, ptr_l, nn);
     int node = 0;                                               // local node index
     int seg_end = __shfl_sync(0xffffffffu, ptr_l, 1);
-    float acc[V];
+    float acc[V], racc[V];
 #pragma unroll
-    for (int c = 0; c < V; ++c) acc[c] = 0.f;
+    for (int c = 0; c < V; ++c) acc[c] = racc[c] = 0.f;
 #define OCCU_FLUSH_NODE(nd)                                                                  \
   do {                                                                                       \
     const int deg_ = __shfl_sync(0xffffffffu, ptr_l, (nd) + 1) - __shfl_sync(0xffffffffu, ptr_l, (nd)); \
-    float *o_ = h_out + (t0 + (nd)) * D + lane * V;                                          \
-    _Pragma("unroll") for (int c = 0; c < V; ++c) {                                          \
-      float a_ = acc[c];                                                                     \
-      if (mean) a_ = a_ / float(deg_ > 0 ? deg_ : 1);                                        \
-      o_[c] = lrelu(a_, slope);                                                              \
-      acc[c] = 0.f;                                                                          \
+    if constexpr (!RP) {                                                                     \
+      float *o_ = h_out + (t0 + (nd)) * D + lane * V;                                        \
+      _Pragma("unroll") for (int c = 0; c < V; ++c) {                                        \
+        float a_ = acc[c];                                                                   \
+        if (mean) a_ = a_ / float(deg_ > 0 ? deg_ : 1);                                      \
+        o_[c] = lrelu(a_, slope);                                                            \
+        acc[c] = 0.f;                                                                        \
+      }                                                                                      \
+    } else {                                                                                 \
+      float o_[V];                                                                           \
+      _Pragma("unroll") for (int c = 0; c < V; ++c) {                                        \
+        float a_ = acc[c];                                                                   \
+        if (mean) a_ = a_ / float(deg_ > 0 ? deg_ : 1);                                      \
+        o_[c] = lrelu(a_, slope);                                                            \
+        acc[c] = 0.f;                                                                        \
+      }                                                                                      \
+      if (h_out) store_row<V>(h_out + (t0 + (nd)) * D + lane * V, o_);                       \
+      const int gcur_ = __shfl_sync(0xffffffffu, gr_l, (nd));                                \
+      const int gnxt_ = __shfl_sync(0xffffffffu, gr_l, ((nd) + 1) & 31);                     \
+      _Pragma("unroll") for (int c = 0; c < V; ++c) racc[c] += o_[c];                        \
+      if ((nd) + 1 >= nn || gnxt_ != gcur_) {                                                \
+        store_row<V>(rpart + (t0 + (nd)) * D + lane * V, racc);                              \
+        _Pragma("unroll") for (int c = 0; c < V; ++c) racc[c] = 0.f;                         \
+      }                                                                                      \
     }                                                                                        \
   } while (0)
     for (int base = e_beg; base < e_end; base += 32) {
@@ -354,6 +388,131 @@ __global__ void __launch_bounds__(NT) gather_segsum_kernel(
   }
 }
 
+// Variant with deeper memory-level parallelism (same arithmetic and summation order
+// as gather_segsum_kernel): persistent warps walk chunks of NPW destinations; each
+// group issues G gathered (g, h̄[s]) row pairs unconditionally (indices clamped into
+// the chunk, surplus rows are never accumulated), and the next chunk's in_ptr /
+// in_src words are requested while the current chunk is summed.
+template <int D, int G, bool RP>
+__global__ void __launch_bounds__(NT, G == 4 ? 4 : 3) gather_segsum_v2_kernel(
+    const float *__restrict__ g, const float *__restrict__ hbar,
+    const int32_t *__restrict__ in_ptr, const int32_t *__restrict__ in_src, int N, int mean,
+    float slope, float *__restrict__ h_out, const int32_t *__restrict__ node_graph,
+    float *__restrict__ rpart) {
+  constexpr int V = D / 32;
+  constexpr int NPW = 8;
+  const int lane = threadIdx.x & 31;
+  const long nw = (long(gridDim.x) * NT) / 32;
+  long t0 = (blockIdx.x * long(NT) + threadIdx.x) / 32 * NPW;
+  if (t0 >= N) return;
+  auto load_ptr = [&](long t) {
+    const int n = int(min(long(NPW), N - t));
+    return lane <= n ? __ldg(in_ptr + t + lane) : 0;
+  };
+  int ptr_l = load_ptr(t0);
+  int s_first = 0;
+  {
+    const int eb = __shfl_sync(0xffffffffu, ptr_l, 0);
+    const int n = int(min(long(NPW), N - t0));
+    const int ee = __shfl_sync(0xffffffffu, ptr_l, n);
+    s_first = eb + lane < ee ? __ldg(in_src + eb + lane) : 0;
+  }
+  for (; t0 < N; t0 += nw * NPW) {
+    const int nn = int(min(long(NPW), N - t0));
+    const long t1 = t0 + nw * NPW;
+    const int ptr_n = t1 < N ? load_ptr(t1) : 0;             // next chunk, in flight now
+    const int gr_l = (RP && lane < nn) ? __ldg(node_graph + t0 + lane) : -1;
+    const int e_beg = __shfl_sync(0xffffffffu, ptr_l, 0);
+    const int e_end = __shfl_sync(0xffffffffu, ptr_l, nn);
+    int node = 0;
+    int seg_end = __shfl_sync(0xffffffffu, ptr_l, 1);
+    float acc[V], racc[V];
+#pragma unroll
+    for (int c = 0; c < V; ++c) acc[c] = racc[c] = 0.f;
+    auto flush = [&](int nd) {
+      const int deg = __shfl_sync(0xffffffffu, ptr_l, nd + 1) - __shfl_sync(0xffffffffu, ptr_l, nd);
+      float o[V];
+#pragma unroll
+      for (int c = 0; c < V; ++c) {
+        float x = acc[c];
+        if (mean) x = x / float(deg > 0 ? deg : 1);
+        o[c] = lrelu(x, slope);
+        acc[c] = 0.f;
+      }
+      if (!RP || h_out) store_row<V>(h_out + (t0 + nd) * D + lane * V, o);
+      if (RP) {
+        const int gc = __shfl_sync(0xffffffffu, gr_l, nd);
+        const int gn = __shfl_sync(0xffffffffu, gr_l, (nd + 1) & 31);
+#pragma unroll
+        for (int c = 0; c < V; ++c) racc[c] += o[c];
+        if (nd + 1 >= nn || gn != gc) {
+          store_row<V>(rpart + (t0 + nd) * D + lane * V, racc);
+#pragma unroll
+          for (int c = 0; c < V; ++c) racc[c] = 0.f;
+        }
+      }
+    };
+    int s_l = s_first;
+    int s_next = 0;
+    bool next_src_issued = false;
+    for (int base = e_beg; base < e_end; base += 32) {
+      const int cnt = min(32, e_end - base);
+      if (base > e_beg) s_l = lane < cnt ? __ldg(in_src + base + lane) : 0;
+      for (int j = 0; j < cnt; j += G) {
+        float gv[G][V], hv[G][V];
+#pragma unroll
+        for (int u = 0; u < G; ++u) {
+          const int kk = min(j + u, cnt - 1);
+          const int sidx = __shfl_sync(0xffffffffu, s_l, kk);
+          const float *gr = g + long(base + kk) * D + lane * V;
+          const float *hr = hbar + long(sidx) * D + lane * V;
+          if constexpr (V == 4) {
+            const float4 a = __ldg(reinterpret_cast<const float4 *>(gr));
+            const float4 b = __ldg(reinterpret_cast<const float4 *>(hr));
+            gv[u][0] = a.x; gv[u][1 % V] = a.y; gv[u][2 % V] = a.z; gv[u][3 % V] = a.w;
+            hv[u][0] = b.x; hv[u][1 % V] = b.y; hv[u][2 % V] = b.z; hv[u][3 % V] = b.w;
+          } else {
+#pragma unroll
+            for (int c = 0; c < V; ++c) {
+              gv[u][c] = __ldg(gr + c);
+              hv[u][c] = __ldg(hr + c);
+            }
+          }
+        }
+        if (!next_src_issued && t1 < N) {                      // next chunk's first sources
+          const int nb = __shfl_sync(0xffffffffu, ptr_n, 0);
+          const int n1 = int(min(long(NPW), N - t1));
+          const int ne = __shfl_sync(0xffffffffu, ptr_n, n1);
+          s_next = nb + lane < ne ? __ldg(in_src + nb + lane) : 0;
+          next_src_issued = true;
+        }
+#pragma unroll
+        for (int u = 0; u < G; ++u) {
+          if (j + u < cnt) {
+            const int k = base + j + u;
+            while (k >= seg_end) {
+              flush(node);
+              ++node;
+              seg_end = __shfl_sync(0xffffffffu, ptr_l, node + 1);
+            }
+#pragma unroll
+            for (int c = 0; c < V; ++c) acc[c] = fmaf(gv[u][c], hv[u][c], acc[c]);
+          }
+        }
+      }
+    }
+    for (; node < nn; ++node) flush(node);
+    if (!next_src_issued && t1 < N) {
+      const int nb = __shfl_sync(0xffffffffu, ptr_n, 0);
+      const int n1 = int(min(long(NPW), N - t1));
+      const int ne = __shfl_sync(0xffffffffu, ptr_n, n1);
+      s_next = nb + lane < ne ? __ldg(in_src + nb + lane) : 0;
+    }
+    ptr_l = ptr_n;
+    s_first = s_next;
+  }
+}
+
 // e0[k] = edge_feat[in_eid[k]]  (a1)
 __global__ void permute_rows_kernel(const float *__restrict__ src, const int32_t *__restrict__ idx,
                                     int rows, int width, float *__restrict__ dst) {
@@ -374,7 +533,10 @@ __global__ void readout_head_kernel(const float *__restrict__ h, const int32_t *
                                     const float *__restrict__ b_1, const float *__restrict__ w_2,
                                     const float *__restrict__ b_2, float slope,
                                     float *__restrict__ r_out, float *__restrict__ c_out,
-                                    float *__restrict__ yhat) {
+                                    float *__restrict__ yhat, int chunk) {
+  // chunk == 0: h holds the node states, summed u0 + grp, u0 + grp + 4, ...
+  // chunk > 0: h holds gather_segsum_kernel's chunk partials; graph b's rows are
+  // min(u1 - 1, chunk*c + chunk - 1) for chunks c = u0/chunk .. (u1-1)/chunk.
   extern __shared__ float sm[];
   float *part = sm;              // [4][D]
   float *rs = part + 4 * D;      // [D]
@@ -383,7 +545,12 @@ __global__ void readout_head_kernel(const float *__restrict__ h, const int32_t *
   const int u0 = node_off[b], u1 = node_off[b + 1];
   const int c = threadIdx.x % D, grp = threadIdx.x / D;   // blockDim = 4*D
   float acc = 0.f;
-  for (int u = u0 + grp; u < u1; u += 4) acc += h[long(u) * D + c];
+  if (chunk > 0) {
+    for (int k = u0 / chunk + grp; k <= (u1 - 1) / chunk; k += 4)
+      acc += h[long(min(u1 - 1, k * chunk + chunk - 1)) * D + c];
+  } else {
+    for (int u = u0 + grp; u < u1; u += 4) acc += h[long(u) * D + c];
+  }
   part[grp * D + c] = acc;
   __syncthreads();
   if (threadIdx.x < D) {
@@ -393,18 +560,27 @@ __global__ void readout_head_kernel(const float *__restrict__ h, const int32_t *
     r_out[long(b) * D + c] = rv;
   }
   __syncthreads();
-  for (int j = threadIdx.x; j < d_h; j += blockDim.x) {
+  // head (a8): warp per hidden unit j, lanes over k (coalesced W_1 rows), fixed
+  // butterfly reduction order
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, nwarp = blockDim.x >> 5;
+  for (int j = warp; j < d_h; j += nwarp) {
     float cv = 0.f;
-    for (int k = 0; k < D; ++k) cv = fmaf(W_1[long(j) * D + k], rs[k], cv);
-    cv += b_1[j];
-    c_out[long(b) * d_h + j] = cv;
-    os[j] = lrelu(cv, slope);
+    for (int k = lane; k < D; k += 32) cv = fmaf(__ldg(W_1 + long(j) * D + k), rs[k], cv);
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) cv += __shfl_xor_sync(0xffffffffu, cv, o);
+    if (lane == 0) {
+      cv += b_1[j];
+      c_out[long(b) * d_h + j] = cv;
+      os[j] = lrelu(cv, slope);
+    }
   }
   __syncthreads();
-  if (threadIdx.x == 0) {
+  if (warp == 0) {
     float y = 0.f;
-    for (int j = 0; j < d_h; ++j) y = fmaf(w_2[j], os[j], y);
-    yhat[b] = y + b_2[0];
+    for (int j = lane; j < d_h; j += 32) y = fmaf(__ldg(w_2 + j), os[j], y);
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) y += __shfl_xor_sync(0xffffffffu, y, o);
+    if (lane == 0) yhat[b] = y + b_2[0];
   }
 }
 
@@ -931,9 +1107,9 @@ static int forward_layer_impl(const occu_ctx *ctx, const DevCsr &csr, const FwdL
   }
   if (csr.N > 0) {
     OCCU_PROF_BEGIN(ctx, "gather_segsum", st);
-    gather_segsum_kernel<D><<<grid_for(long(csr.N) * 4, NT, 16 * sms), NT, 0, st>>>(
+    gather_segsum_kernel<D, false><<<grid_for(long(csr.N) * 4, NT, 16 * sms), NT, 0, st>>>(
         a.g, a.hbar, csr.in_ptr, csr.in_src, csr.N, ctx->cfg.aggr == OCCU_AGGR_MEAN,
-        ctx->cfg.slope, a.h_out);
+        ctx->cfg.slope, a.h_out, nullptr, nullptr);
     OCCU_PROF_END(ctx);
     LAUNCH_CHECK();
     ++n;
@@ -943,22 +1119,44 @@ static int forward_layer_impl(const occu_ctx *ctx, const DevCsr &csr, const FwdL
 
 template <int D>
 static int gather_impl(const occu_ctx *ctx, const DevCsr &csr, const float *g, const float *hbar,
-                       float *h_out, cudaStream_t st) {
+                       float *h_out, float *rpart, cudaStream_t st) {
   if (csr.N <= 0) return 0;
+  static const int variant = [] {
+    const char *e = getenv("OCCU_GATHER_V");
+    return e ? atoi(e) : 1;
+  }();
+  static const int occ = [] {
+    const char *e = getenv("OCCU_GATHER_BPS");
+    return e ? atoi(e) : 8;
+  }();
+  const int mean = ctx->cfg.aggr == OCCU_AGGR_MEAN;
   OCCU_PROF_BEGIN(ctx, "gather_segsum", st);
-  gather_segsum_kernel<D><<<grid_for(long(csr.N) * 4, NT, 16 * ctx->num_sms), NT, 0, st>>>(
-      g, hbar, csr.in_ptr, csr.in_src, csr.N, ctx->cfg.aggr == OCCU_AGGR_MEAN, ctx->cfg.slope,
-      h_out);
+#define OCCU_GATHER_ARGS g, hbar, csr.in_ptr, csr.in_src, csr.N, mean, ctx->cfg.slope, h_out, csr.node_graph, rpart
+  if (variant == 0) {
+    const int grid = grid_for(long(csr.N) * 4, NT, 16 * ctx->num_sms);
+    if (rpart) gather_segsum_kernel<D, true><<<grid, NT, 0, st>>>(OCCU_GATHER_ARGS);
+    else gather_segsum_kernel<D, false><<<grid, NT, 0, st>>>(OCCU_GATHER_ARGS);
+  } else {
+    const int grid = grid_for(long(csr.N) * 4, NT, occ * ctx->num_sms);
+    if (variant == 1) {
+      if (rpart) gather_segsum_v2_kernel<D, 4, true><<<grid, NT, 0, st>>>(OCCU_GATHER_ARGS);
+      else gather_segsum_v2_kernel<D, 4, false><<<grid, NT, 0, st>>>(OCCU_GATHER_ARGS);
+    } else {
+      if (rpart) gather_segsum_v2_kernel<D, 8, true><<<grid, NT, 0, st>>>(OCCU_GATHER_ARGS);
+      else gather_segsum_v2_kernel<D, 8, false><<<grid, NT, 0, st>>>(OCCU_GATHER_ARGS);
+    }
+  }
+#undef OCCU_GATHER_ARGS
   OCCU_PROF_END(ctx);
   LAUNCH_CHECK();
   return 1;
 }
 
 int launch_gather_segsum(const occu_ctx *ctx, const DevCsr &csr, const float *g,
-                         const float *hbar, float *h_out, cudaStream_t st) {
+                         const float *hbar, float *h_out, float *rpart, cudaStream_t st) {
   switch (ctx->cfg.d) {
-    case 64: return gather_impl<64>(ctx, csr, g, hbar, h_out, st);
-    case 128: return gather_impl<128>(ctx, csr, g, hbar, h_out, st);
+    case 64: return gather_impl<64>(ctx, csr, g, hbar, h_out, rpart, st);
+    case 128: return gather_impl<128>(ctx, csr, g, hbar, h_out, rpart, st);
     default: return -int(cudaErrorInvalidValue);
   }
 }
@@ -983,7 +1181,7 @@ int launch_permute_rows(const occu_ctx *ctx, const float *src, const int32_t *id
   return 1;
 }
 
-int launch_readout_head(const occu_ctx *ctx, const DevCsr &csr, const float *h,
+int launch_readout_head(const occu_ctx *ctx, const DevCsr &csr, const float *h, bool chunked,
                         const float *params, float *r, float *c, float *yhat, cudaStream_t st) {
   const occu_config &cf = ctx->cfg;
   const ParamLayout &L = ctx->layout;
@@ -992,7 +1190,7 @@ int launch_readout_head(const occu_ctx *ctx, const DevCsr &csr, const float *h,
   readout_head_kernel<<<csr.B, 4 * cf.d, smem, st>>>(h, csr.node_off, cf.d, cf.d_h,
                                                       params + L.W_1, params + L.b_1,
                                                       params + L.w_2, params + L.b_2, cf.slope,
-                                                      r, c, yhat);
+                                                      r, c, yhat, chunked ? 8 : 0);
   OCCU_PROF_END(ctx);
   LAUNCH_CHECK();
   return 1;

@@ -113,6 +113,7 @@ struct RowGemmArgs {
   int mean;
   float *dal;              // EDGEBWD: dα [R]
   float *part;             // GATEAGG: [R/32 units][2 slots][D] boundary-segment partials
+  int rev;                 // walk tiles last-to-first (reads what the previous kernel wrote last, still in L2)
 };
 
 struct Smem {
@@ -214,6 +215,11 @@ __device__ __forceinline__ void warp_store_chunk(float *buf, float *__restrict__
   }
 }
 
+__device__ __forceinline__ int tile_of(const RowGemmArgs &a, int tiles, int i) {
+  const int t = int(blockIdx.x) + i * int(gridDim.x);
+  return a.rev ? tiles - 1 - t : t;
+}
+
 __device__ __forceinline__ void group_bar(int g) {
   asm volatile("bar.sync %0, 256;" ::"r"(1 + g) : "memory");
 }
@@ -288,7 +294,7 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
       }
       for (int i = 0; i < my; ++i) {
         const int j = i & 1;
-        const int r0 = int(blockIdx.x + i * gridDim.x) * TM;
+        const int r0 = tile_of(a, tiles, i) * TM;
         TT_WAIT_BEGIN
         if (i >= 2) tc::mbar_wait(s.empty + j, ((i >> 1) - 1) & 1);
         TT_WAIT_END
@@ -345,7 +351,7 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
     TT_DECL
     for (int i = 0; i < my; ++i) {
       const int j = i & 1;
-      const long r0 = long(blockIdx.x + i * gridDim.x) * TM;
+      const long r0 = long(tile_of(a, tiles, i)) * TM;
       const bool live = row < min(TM, int(a.R - r0));
       TT_WAIT_BEGIN
       tc::mbar_wait(s.full + j, (i >> 1) & 1);
@@ -410,7 +416,7 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
     TT_DECL
     for (int i = g; i < my; i += 2) {
       const int j = i & 1;
-      const long r0 = long(blockIdx.x + i * gridDim.x) * TM;
+      const long r0 = long(tile_of(a, tiles, i)) * TM;
       const int nrows = min(TM, int(a.R - r0));
       const bool live = row < nrows;
       float aux = 0.f;
@@ -820,52 +826,76 @@ __global__ void __launch_bounds__(256) wimage_kernel(const WImageJob *__restrict
   }
 }
 
-// Layer-1 edge transform (F_e small, e.g. 4): e' = σ(α · W_e e) on CUDA cores,
-// one warp per edge, lanes over 4-channel groups (coalesced 512-byte rows).
+// Layer-1 edge transform (F_e small, e.g. 4): e' = σ(α · W_e e) on CUDA cores (a3).
+// A warp takes 32 consecutive in-CSR edges per iteration: lane j loads edge j's
+// indices, α = p[src] + q[dst] and its Ke input features (one independent gather
+// chain per lane, all 32 in flight), then the warp walks the 32 edges, broadcasting
+// α and e by shuffle; each lane computes D/32 channels of the edge's row
+// (coalesced row stores).  With eid != null the input row of in-CSR edge k is
+// e_in[eid[k]] (a1's permutation fused in); e0_out, if set, receives the permuted
+// rows (kept for the backward).  Ke <= KM <= 16.
 template <int D, int KM>
 __global__ void __launch_bounds__(256) edge_small_kernel(
     const float *__restrict__ e_in, int Ke, const float *__restrict__ W_e,
     const float *__restrict__ p, const float *__restrict__ q, const int32_t *__restrict__ in_src,
-    const int32_t *__restrict__ in_dst, int E, float *__restrict__ e_out) {
-  // One warp per 4 consecutive edges (4 independent index/α chains in flight),
-  // lanes over 4-channel groups: coalesced 512-byte rows.  Ke <= 16.
-  extern __shared__ float wsm[];            // [Ke][D] = W_eᵀ (conflict-free float4 reads)
+    const int32_t *__restrict__ in_dst, const int32_t *__restrict__ eid, int E,
+    float *__restrict__ e_out, float *__restrict__ e0_out) {
+  constexpr int V = D / 32;                 // channels per lane
+  extern __shared__ float wsm[];            // [Ke][D] = W_eᵀ
   for (int i = threadIdx.x; i < D * Ke; i += blockDim.x) wsm[(i % Ke) * D + i / Ke] = W_e[i];
   __syncthreads();
-  constexpr int G = D / 4;                  // lanes per edge row
-  constexpr int RPI = 32 / G;               // rows per warp instruction
-  constexpr int EPW = 4 * RPI;              // edges per warp iteration
   const int lane = threadIdx.x & 31;
-  const int sub = lane / G, c = (lane % G) * 4;
+  const int c = lane * V;
+  float w[KM][V];                           // this lane's W_e columns, in registers
+#pragma unroll
+  for (int j = 0; j < KM; ++j)
+#pragma unroll
+    for (int v = 0; v < V; ++v) w[j][v] = j < Ke ? wsm[j * D + c + v] : 0.f;
   const long nwarps = long(gridDim.x) * (blockDim.x / 32);
-  for (long k0 = (blockIdx.x * long(blockDim.x / 32) + threadIdx.x / 32) * EPW; k0 < E;
-       k0 += nwarps * EPW) {
-    float al[4], ev[4][KM];
+  for (long k0 = (blockIdx.x * long(blockDim.x / 32) + threadIdx.x / 32) * 32; k0 < E;
+       k0 += nwarps * 32) {
+    const long k = k0 + lane;
+    const int cnt = int(min(32L, E - k0));
+    float al = 0.f, ev[KM];
 #pragma unroll
-    for (int u = 0; u < 4; ++u) {
-      const long k = k0 + u * RPI + sub;
-      al[u] = 0.f;
-      if (k < E) al[u] = __ldg(p + in_src[k]) + __ldg(q + in_dst[k]);
+    for (int j = 0; j < KM; ++j) ev[j] = 0.f;
+    if (k < E) {
+      al = __ldg(p + __ldg(in_src + k)) + __ldg(q + __ldg(in_dst + k));
+      const long row = eid ? long(__ldg(eid + k)) : k;
+      if (KM == 4 && Ke == 4) {
+        const float4 x = __ldg(reinterpret_cast<const float4 *>(e_in + row * 4));
+        ev[0] = x.x; ev[1 % KM] = x.y; ev[2 % KM] = x.z; ev[3 % KM] = x.w;
+      } else {
 #pragma unroll
-      for (int j = 0; j < KM; ++j) ev[u][j] = (j < Ke && k < E) ? __ldg(e_in + k * Ke + j) : 0.f;
+        for (int j = 0; j < KM; ++j) ev[j] = j < Ke ? __ldg(e_in + row * Ke + j) : 0.f;
+      }
+      if (e0_out) {
+#pragma unroll
+        for (int j = 0; j < KM; ++j)
+          if (j < Ke) e0_out[k * Ke + j] = ev[j];
+      }
     }
+    for (int u = 0; u < cnt; ++u) {
+      const float a = __shfl_sync(0xffffffffu, al, u);
+      float z[V];
 #pragma unroll
-    for (int u = 0; u < 4; ++u) {
-      const long k = k0 + u * RPI + sub;
-      float z[4] = {0.f, 0.f, 0.f, 0.f};
+      for (int v = 0; v < V; ++v) z[v] = 0.f;
 #pragma unroll
-      for (int j = 0; j < KM; ++j)
-        if (j < Ke) {
-          const float4 w = *reinterpret_cast<const float4 *>(wsm + j * D + c);
-          z[0] = fmaf(w.x, ev[u][j], z[0]);
-          z[1] = fmaf(w.y, ev[u][j], z[1]);
-          z[2] = fmaf(w.z, ev[u][j], z[2]);
-          z[3] = fmaf(w.w, ev[u][j], z[3]);
-        }
-      float o[4];
+      for (int j = 0; j < KM; ++j) {
+        const float x = __shfl_sync(0xffffffffu, ev[j], u);
 #pragma unroll
-      for (int t = 0; t < 4; ++t) o[t] = fast_rcp(1.f + fast_exp(-(al[u] * z[t])));
-      if (k < E) *reinterpret_cast<float4 *>(e_out + k * D + c) = make_float4(o[0], o[1], o[2], o[3]);
+        for (int v = 0; v < V; ++v) z[v] = fmaf(w[j][v], x, z[v]);
+      }
+      float o[V];
+#pragma unroll
+      for (int v = 0; v < V; ++v) o[v] = fast_rcp(1.f + fast_exp(-(a * z[v])));
+      float *dst = e_out + (k0 + u) * D + c;
+      if constexpr (V == 4) {
+        *reinterpret_cast<float4 *>(dst) = make_float4(o[0], o[1], o[2], o[3]);
+      } else {
+#pragma unroll
+        for (int v = 0; v < V; v += 2) *reinterpret_cast<float2 *>(dst + v) = make_float2(o[v], o[v + 1]);
+      }
     }
   }
 }
@@ -1206,19 +1236,22 @@ static int tc_forward_layer_impl(const occu_ctx *ctx, const DevCsr &csr, int lay
   ra.A = a.h_in; ra.K = a.K; ra.R = csr.N; ra.W = a.W_u; ra.out = a.hbar;
   ra.wimg = tc_wimg(ctx, 0, layer); ra.wfexp = tc_wfexp(ctx, 0, layer);
   ra.a_s = a.a_s; ra.a_d = a.a_d; ra.p = a.p; ra.q = a.q;
+  // L2 reuse: node and gate walk their rows last-to-first, so each kernel starts on the
+  // rows its producer (gather resp. edge transform, both first-to-last) wrote last
+  ra.rev = ctx->l2_order;
   if ((r = launch_rowgemm<D, EPI_NODE>(ctx, ra, "node_tc", st)) < 0) return r;
   n += r;
   if (csr.E > 0) {
     // a3: edge transform
     if (a.Ke <= 16) {
-      const int grid = int(std::min<long>((long(csr.E) * (D / 4) / 4 + 255) / 256, 8L * ctx->num_sms));
+      const int grid = int(std::min<long>((long(csr.E) + 255) / 256, 8L * ctx->num_sms));
       OCCU_PROF_BEGIN(ctx, "edge_small", st);
       if (a.Ke <= 4)
-        edge_small_kernel<D, 4><<<grid, 256, D * a.Ke * 4, st>>>(a.e_in, a.Ke, a.W_e, a.p, a.q,
-                                                                 csr.in_src, csr.in_dst, csr.E, a.e_out);
+        edge_small_kernel<D, 4><<<grid, 256, D * a.Ke * 4, st>>>(
+            a.e_in, a.Ke, a.W_e, a.p, a.q, csr.in_src, csr.in_dst, a.e_eid, csr.E, a.e_out, a.e0_out);
       else
-        edge_small_kernel<D, 16><<<grid, 256, D * a.Ke * 4, st>>>(a.e_in, a.Ke, a.W_e, a.p, a.q,
-                                                                  csr.in_src, csr.in_dst, csr.E, a.e_out);
+        edge_small_kernel<D, 16><<<grid, 256, D * a.Ke * 4, st>>>(
+            a.e_in, a.Ke, a.W_e, a.p, a.q, csr.in_src, csr.in_dst, a.e_eid, csr.E, a.e_out, a.e0_out);
       OCCU_PROF_END(ctx);
       TC_CHECK();
       ++n;
@@ -1247,6 +1280,7 @@ static int tc_forward_layer_impl(const occu_ctx *ctx, const DevCsr &csr, int lay
       rg.slope = slope;
       rg.A = a.e_out; rg.K = D; rg.R = csr.E; rg.W = a.W_m; rg.out = a.g;
       rg.wimg = tc_wimg(ctx, 2, layer); rg.wfexp = tc_wfexp(ctx, 2, layer);
+      rg.rev = ctx->l2_order;
       if ((r = launch_rowgemm<D, EPI_GATE>(ctx, rg, "gate_tc", st)) < 0) return r;
       n += r;
     }
@@ -1263,7 +1297,7 @@ static int tc_forward_layer_impl(const occu_ctx *ctx, const DevCsr &csr, int lay
     }
   } else {
     // a5 + a6: gather + segmented sum (CUDA cores, warp per 8 destinations)
-    if ((r = launch_gather_segsum(ctx, csr, a.g, a.hbar, a.h_out, st)) < 0) return r;
+    if ((r = launch_gather_segsum(ctx, csr, a.g, a.hbar, a.h_out, a.rpart, st)) < 0) return r;
     n += r;
   }
   return n;

@@ -43,6 +43,7 @@ struct Workspace {
   DevBuf e0;               // edge features permuted to in-CSR order [E][F_e]
   std::vector<DevBuf> hbar, p, q, e, h;   // per layer
   DevBuf g;                // [E][d] channel-softmax gates (scratch)
+  DevBuf rpart;            // [N][d] readout chunk partials (rows written sparsely) when h_L is kept
   DevBuf r, c, yhat;       // [B][d], [B][d_h], [B]
   // backward scratch
   DevBuf dy, dc, dr, dh, dhprev, dP, MG, DV, DZ, deA, deB, dalpha, dpq, partial, loss;
@@ -88,6 +89,7 @@ struct occu_ctx {
   bool weights_ready = false;
   bool keep = false;
   int path = 0;            // 0: tensor cores, 1: CUDA-core SIMT FP32, 2: tensor cores + fused aggregation
+  int l2_order = 1;        // alternate row-walk direction between producer/consumer kernels (L2 reuse)
   occu::DevBuf wimg, wjobs, wfexp;   // prebuilt tensor-core weight images (per parameter version)
   int64_t params_version = 0, wimg_version = -1;
   float weight_decay = 1e-4f;
@@ -96,6 +98,7 @@ struct occu_ctx {
   occu::Workspace ws;
   occu::DevCsr last_csr;   // geometry of the last forward (for occu_get_tensor)
   bool have_forward = false;
+  bool h_last_stored = true;   // false: the last forward kept only readout partials of h_L
   int64_t launches = 0;
   mutable occu::Profiler prof;
   // data parallel
@@ -117,6 +120,11 @@ struct FwdLayerArgs {
   const float *e_in; int Ke;           // [E][Ke] in-CSR order
   const float *W_u, *W_e, *W_m, *a_s, *a_d;
   float *hbar, *p, *q, *e_out, *g, *h_out;   // e_out may be null
+  // Fused variants (tensor-core path): layer 1 reads edge_feat rows through in_eid
+  // (e_eid != null; e0_out, if set, receives the permuted copy for the backward), and
+  // the last layer's aggregation emits readout chunk partials into rpart (h_out may
+  // then be null).  See gather_segsum_kernel / readout_head_kernel.
+  const int32_t *e_eid; float *e0_out; float *rpart;
 };
 int launch_forward_layer(const occu_ctx *ctx, const DevCsr &csr, const FwdLayerArgs &a,
                          cudaStream_t st);
@@ -141,10 +149,12 @@ size_t tc_partial_floats(int E, int D);
 int launch_forward_layer_tc(const occu_ctx *ctx, const DevCsr &csr, int layer, const FwdLayerArgs &a,
                             float *partial, cudaStream_t st);
 int launch_gather_segsum(const occu_ctx *ctx, const DevCsr &csr, const float *g,
-                         const float *hbar, float *h_out, cudaStream_t st);
+                         const float *hbar, float *h_out, float *rpart, cudaStream_t st);
 int launch_permute_rows(const occu_ctx *ctx, const float *src, const int32_t *idx, int rows,
                         int width, float *dst, cudaStream_t st);
-int launch_readout_head(const occu_ctx *ctx, const DevCsr &csr, const float *h,
+// h: [N][d] last-layer states, or (chunked) the readout chunk partials of
+// gather_segsum_kernel (row min(u1 - 1, 8c + 7) holds graph b's sum over chunk c).
+int launch_readout_head(const occu_ctx *ctx, const DevCsr &csr, const float *h, bool chunked,
                         const float *params, float *r, float *c, float *yhat, cudaStream_t st);
 
 struct BwdLayerArgs {

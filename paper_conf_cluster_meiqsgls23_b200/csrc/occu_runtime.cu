@@ -226,31 +226,53 @@ occu_status forward(occu_ctx *ctx, const DevCsr &csr, const float *nf, const flo
   if (st != OCCU_OK) return st;
   cudaStream_t s = ctx->stream;
   const float *P = ctx->params.as<float>();
-  LK(launch_permute_rows(ctx, ef, csr.in_eid, csr.E, c.F_e, w.e0.as<float>(), s), "permute e0");
-  if (ctx->path != 1 && tc_supported(c)) LK(tc_prepare_weights(ctx, s), "weight images");
+  const bool tc = ctx->path != 1 && tc_supported(c);
+  // Tensor-core path fusions: a1's edge permutation folded into the layer-1 edge kernel,
+  // and the readout's node sums folded into the last aggregation (chunk partials).
+  const bool fuse_e0 = tc && c.F_e <= 16;
+  const bool fuse_ro = tc && ctx->path == 0;
+  if (!fuse_e0) LK(launch_permute_rows(ctx, ef, csr.in_eid, csr.E, c.F_e, w.e0.as<float>(), s), "permute e0");
+  if (tc) LK(tc_prepare_weights(ctx, s), "weight images");
+  float *rpart = nullptr;
+  if (fuse_ro) {
+    if (save_all) {
+      CK(w.rpart.ensure(size_t(csr.N) * c.d * 4), "alloc rpart");
+      rpart = w.rpart.as<float>();
+    } else {
+      rpart = w.h[c.L - 1].as<float>();     // h_L itself is not stored in this mode
+    }
+  }
   for (int i = 0; i < c.L; ++i) {
+    const bool last = i == c.L - 1;
     FwdLayerArgs a{};
     a.h_in = i == 0 ? nf : w.h[i - 1].as<float>();
     a.K = L.d_in[i];
-    a.e_in = i == 0 ? w.e0.as<float>() : w.e[i - 1].as<float>();
+    a.e_in = i == 0 ? (fuse_e0 ? ef : w.e0.as<float>()) : w.e[i - 1].as<float>();
+    a.e_eid = (i == 0 && fuse_e0) ? csr.in_eid : nullptr;
+    a.e0_out = (i == 0 && fuse_e0 && save_all) ? w.e0.as<float>() : nullptr;
     a.Ke = L.de_in[i];
     a.W_u = P + L.W_u[i]; a.W_e = P + L.W_e[i]; a.W_m = P + L.W_m[i];
     a.a_s = P + L.a_s[i]; a.a_d = P + L.a_d[i];
     a.hbar = w.hbar[i].as<float>(); a.p = w.p[i].as<float>(); a.q = w.q[i].as<float>();
-    a.e_out = (i < c.L - 1 || save_all) ? w.e[i].as<float>() : nullptr;
+    a.e_out = (!last || save_all) ? w.e[i].as<float>() : nullptr;
     a.g = w.g.as<float>();
     a.h_out = w.h[i].as<float>();
-    if (ctx->path != 1 && tc_supported(c)) {
+    if (tc) {
       a.e_out = w.e[i].as<float>();            // the gate kernel re-reads e'
+      if (last && fuse_ro) {
+        a.rpart = rpart;
+        if (!save_all) a.h_out = nullptr;
+      }
       CK(w.tcpart.ensure(tc_partial_floats(csr.E, c.d) * 4), "alloc tc partials");
       LK(launch_forward_layer_tc(ctx, csr, i, a, w.tcpart.as<float>(), s), "forward layer (tc)");
     } else {
       LK(launch_forward_layer(ctx, csr, a, s), "forward layer");
     }
   }
-  LK(launch_readout_head(ctx, csr, w.h[c.L - 1].as<float>(), P, w.r.as<float>(), w.c.as<float>(),
-                         w.yhat.as<float>(), s),
+  LK(launch_readout_head(ctx, csr, fuse_ro ? rpart : w.h[c.L - 1].as<float>(), fuse_ro, P,
+                         w.r.as<float>(), w.c.as<float>(), w.yhat.as<float>(), s),
      "readout/head");
+  ctx->h_last_stored = !fuse_ro || save_all;
   ctx->last_csr = csr;
   ctx->have_forward = true;
   return OCCU_OK;
@@ -372,6 +394,7 @@ occu_status occu_create(occu_ctx **out, const occu_config *cfg, int cuda_device,
   ctx->device = cuda_device;
   ctx->stream = static_cast<cudaStream_t>(cuda_stream);
   cudaDeviceGetAttribute(&ctx->num_sms, cudaDevAttrMultiProcessorCount, cuda_device);
+  if (const char *e = getenv("OCCU_L2_ORDER")) ctx->l2_order = atoi(e);   // A/B switch
   const size_t pb = (ctx->layout.total + 1) * 4;
   if (ctx->params.ensure(pb) != cudaSuccess || ctx->grads.ensure(pb) != cudaSuccess ||
       ctx->adam_m.ensure(pb) != cudaSuccess || ctx->adam_v.ensure(pb) != cudaSuccess) {
@@ -681,7 +704,10 @@ occu_status occu_get_tensor(occu_ctx *ctx, int32_t which, int32_t layer, void *h
       if (layer == ctx->cfg.L - 1 && !ctx->keep)
         return fail(ctx, OCCU_ENOTREADY, "last-layer e not stored (set keep_intermediates)");
       src = w.e[layer].ptr; need = size_t(c.E) * d * 4; break;
-    case OCCU_T_H: src = w.h[layer].ptr; need = size_t(c.N) * d * 4; break;
+    case OCCU_T_H:
+      if (layer == ctx->cfg.L - 1 && !ctx->h_last_stored)
+        return fail(ctx, OCCU_ENOTREADY, "last-layer h not stored (set keep_intermediates)");
+      src = w.h[layer].ptr; need = size_t(c.N) * d * 4; break;
     case OCCU_T_R: src = w.r.ptr; need = size_t(c.B) * d * 4; break;
     case OCCU_T_YHAT: src = w.yhat.ptr; need = size_t(c.B) * 4; break;
     default: return fail(ctx, OCCU_EINVAL, "unknown tensor");

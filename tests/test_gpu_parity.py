@@ -101,6 +101,27 @@ def test_hub_nodes_spanning_many_tiles(path):
     compare_all(m, c, y, ref, pk)
 
 
+@pytest.mark.parametrize("path", [0, 1, 2], ids=["tcgen05", "simt", "tcgen05fused"])
+@pytest.mark.parametrize("max_nodes", [3, 12, 40])
+def test_readout_without_kept_states(path, max_nodes):
+    """Default (no keep_intermediates): path 0 folds the readout's node sums into the
+    last aggregation (8-node chunk partials), so graphs smaller than a chunk, graphs
+    straddling chunks and single-node graphs are all exercised; r and ŷ vs the oracle."""
+    c = mk(2, 64)
+    b = configs.random_dag_batch(57, 500 + max_nodes, max_nodes=max_nodes, hub=True)
+    flat = weights.unit_scale(wcfg(c), weights.init_flat(wcfg(c), 11))
+    m, y, ref, pk = run_both(c, b, flat, keep=False, path=path)
+    assert rel(m.get_tensor(occu.T_R, 0, (pk["num_graphs"], c.d)), ref["r"]) <= TOL
+    yr = ref["yhat"]
+    assert np.all(np.abs(y - yr) <= TOL * np.maximum(np.abs(yr), 1e-2))
+    if path == 0:
+        with pytest.raises(RuntimeError):
+            m.get_tensor(occu.T_H, c.L - 1, (pk["num_nodes"], c.d))
+    m.keep_intermediates(True)
+    y2 = m.predict(occu.pack(b.graphs), b.node_feat, b.edge_feat)
+    assert np.array_equal(y, y2)          # same kernels and summation order either way
+
+
 def test_tc_and_simt_paths_agree():
     c = mk(3, 128)
     b = configs.cfg2(8)
