@@ -131,7 +131,11 @@ def algorithmic_bytes(N, E, B, d=128, F_n=80, F_e=4, L=3, rrows=None):
     else:
         gather += L * s * N * d
         readout = s * N * d + s * B * (2 * d + 1)
+    # fused edge transform + gate (edgegate_kernel): e' written once, never re-read
+    edge_gate = (s * E * F_e + 4 * E + 8 * E + 8 * N + 2 * s * E * d
+                 + (L - 1) * (s * E * d + 8 * E + 8 * N + 2 * s * E * d))
     out = {"node_tc": node, "edge_small": edge_small, "edge_tc": edge_tc, "gate_tc": gate,
+           "edge_gate_tc": edge_gate,
            "gather_segsum": gather, "readout_head": readout,
            # SIMT path kernels
            "node_gemm": node, "edge_fwd": edge_small + edge_tc + gate}

@@ -525,53 +525,86 @@ __global__ void permute_rows_kernel(const float *__restrict__ src, const int32_t
 }
 
 // ---------------------------------------------------------------------------
-// a7 + a8: readout (mean over the graph's nodes, ascending node id per
-// 4-way interleaved partial, partials combined in fixed order) and head.
+// a7 + a8: readout (mean over the graph's nodes) and head, one CTA of 16 warps per
+// graph.  Warp w sums rows w, w+16, ... (lane = D/32 channels, 4 rows in flight);
+// the 16 warp partials are combined in fixed order.  chunk == 0: the rows are the
+// node states h_u; chunk > 0: they are gather_segsum_kernel's chunk partials (graph
+// b's rows are min(u1 - 1, chunk*c + chunk - 1), c = u0/chunk .. (u1-1)/chunk).
+// Head: warp per hidden unit j (lanes over k, coalesced W_1 rows), butterfly sums.
 // ---------------------------------------------------------------------------
-__global__ void readout_head_kernel(const float *__restrict__ h, const int32_t *__restrict__ node_off,
-                                    int D, int d_h, const float *__restrict__ W_1,
-                                    const float *__restrict__ b_1, const float *__restrict__ w_2,
-                                    const float *__restrict__ b_2, float slope,
-                                    float *__restrict__ r_out, float *__restrict__ c_out,
-                                    float *__restrict__ yhat, int chunk) {
-  // chunk == 0: h holds the node states, summed u0 + grp, u0 + grp + 4, ...
-  // chunk > 0: h holds gather_segsum_kernel's chunk partials; graph b's rows are
-  // min(u1 - 1, chunk*c + chunk - 1) for chunks c = u0/chunk .. (u1-1)/chunk.
+constexpr int RO_WARPS = 16;
+template <int D>
+__global__ void __launch_bounds__(RO_WARPS * 32) readout_head_kernel(
+    const float *__restrict__ h, const int32_t *__restrict__ node_off, int d_h,
+    const float *__restrict__ W_1, const float *__restrict__ b_1, const float *__restrict__ w_2,
+    const float *__restrict__ b_2, float slope, float *__restrict__ r_out,
+    float *__restrict__ c_out, float *__restrict__ yhat, int chunk) {
+  constexpr int V = D / 32;
   extern __shared__ float sm[];
-  float *part = sm;              // [4][D]
-  float *rs = part + 4 * D;      // [D]
-  float *os = rs + D;            // [d_h]
+  float *part = sm;                    // [RO_WARPS][D]
+  float *rs = part + RO_WARPS * D;     // [D]
+  float *os = rs + D;                  // [d_h]
   const int b = blockIdx.x;
   const int u0 = node_off[b], u1 = node_off[b + 1];
-  const int c = threadIdx.x % D, grp = threadIdx.x / D;   // blockDim = 4*D
-  float acc = 0.f;
-  if (chunk > 0) {
-    for (int k = u0 / chunk + grp; k <= (u1 - 1) / chunk; k += 4)
-      acc += h[long(min(u1 - 1, k * chunk + chunk - 1)) * D + c];
-  } else {
-    for (int u = u0 + grp; u < u1; u += 4) acc += h[long(u) * D + c];
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int k0 = chunk > 0 ? u0 / chunk : u0, k1 = chunk > 0 ? (u1 - 1) / chunk + 1 : u1;
+  float acc[V];
+#pragma unroll
+  for (int c = 0; c < V; ++c) acc[c] = 0.f;
+  auto row_of = [&](int k) { return chunk > 0 ? min(u1 - 1, k * chunk + chunk - 1) : k; };
+  int k = k0 + warp;
+  for (; k + 3 * RO_WARPS < k1; k += 4 * RO_WARPS) {
+    float x[4][V];
+#pragma unroll
+    for (int t = 0; t < 4; ++t) {
+      const float *src = h + long(row_of(k + t * RO_WARPS)) * D + lane * V;
+#pragma unroll
+      for (int c = 0; c < V; ++c) x[t][c] = __ldg(src + c);
+    }
+#pragma unroll
+    for (int t = 0; t < 4; ++t)
+#pragma unroll
+      for (int c = 0; c < V; ++c) acc[c] += x[t][c];
   }
-  part[grp * D + c] = acc;
+  for (; k < k1; k += RO_WARPS) {
+    const float *src = h + long(row_of(k)) * D + lane * V;
+#pragma unroll
+    for (int c = 0; c < V; ++c) acc[c] += __ldg(src + c);
+  }
+#pragma unroll
+  for (int c = 0; c < V; ++c) part[warp * D + lane * V + c] = acc[c];
   __syncthreads();
   if (threadIdx.x < D) {
-    const float s = ((part[c] + part[D + c]) + part[2 * D + c]) + part[3 * D + c];
-    const float rv = s / float(u1 - u0);
-    rs[c] = rv;
-    r_out[long(b) * D + c] = rv;
+    float sum = 0.f;
+#pragma unroll
+    for (int w = 0; w < RO_WARPS; ++w) sum += part[w * D + threadIdx.x];
+    const float rv = sum / float(u1 - u0);
+    rs[threadIdx.x] = rv;
+    r_out[long(b) * D + threadIdx.x] = rv;
   }
   __syncthreads();
-  // head (a8): warp per hidden unit j, lanes over k (coalesced W_1 rows), fixed
-  // butterfly reduction order
-  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, nwarp = blockDim.x >> 5;
-  for (int j = warp; j < d_h; j += nwarp) {
-    float cv = 0.f;
-    for (int k = lane; k < D; k += 32) cv = fmaf(__ldg(W_1 + long(j) * D + k), rs[k], cv);
+  for (int j0 = warp; j0 < d_h; j0 += 4 * RO_WARPS) {
+    float cv[4];
 #pragma unroll
-    for (int o = 16; o > 0; o >>= 1) cv += __shfl_xor_sync(0xffffffffu, cv, o);
-    if (lane == 0) {
-      cv += b_1[j];
-      c_out[long(b) * d_h + j] = cv;
-      os[j] = lrelu(cv, slope);
+    for (int t = 0; t < 4; ++t) {
+      const int j = j0 + t * RO_WARPS;
+      cv[t] = 0.f;
+      if (j < d_h) {
+#pragma unroll
+        for (int c = 0; c < V; ++c)
+          cv[t] = fmaf(__ldg(W_1 + long(j) * D + lane * V + c), rs[lane * V + c], cv[t]);
+      }
+    }
+#pragma unroll
+    for (int t = 0; t < 4; ++t) {
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) cv[t] += __shfl_xor_sync(0xffffffffu, cv[t], o);
+      const int j = j0 + t * RO_WARPS;
+      if (lane == 0 && j < d_h) {
+        const float v = cv[t] + b_1[j];
+        c_out[long(b) * d_h + j] = v;
+        os[j] = lrelu(v, slope);
+      }
     }
   }
   __syncthreads();
@@ -1185,12 +1218,13 @@ int launch_readout_head(const occu_ctx *ctx, const DevCsr &csr, const float *h, 
                         const float *params, float *r, float *c, float *yhat, cudaStream_t st) {
   const occu_config &cf = ctx->cfg;
   const ParamLayout &L = ctx->layout;
-  const size_t smem = (4 * cf.d + cf.d + cf.d_h) * 4;
+  const size_t smem = (RO_WARPS * cf.d + cf.d + cf.d_h) * 4;
   OCCU_PROF_BEGIN(ctx, "readout_head", st);
-  readout_head_kernel<<<csr.B, 4 * cf.d, smem, st>>>(h, csr.node_off, cf.d, cf.d_h,
-                                                      params + L.W_1, params + L.b_1,
-                                                      params + L.w_2, params + L.b_2, cf.slope,
-                                                      r, c, yhat, chunked ? 8 : 0);
+#define OCCU_RO_ARGS h, csr.node_off, cf.d_h, params + L.W_1, params + L.b_1, params + L.w_2, \
+    params + L.b_2, cf.slope, r, c, yhat, chunked ? 8 : 0
+  if (cf.d == 64) readout_head_kernel<64><<<csr.B, RO_WARPS * 32, smem, st>>>(OCCU_RO_ARGS);
+  else readout_head_kernel<128><<<csr.B, RO_WARPS * 32, smem, st>>>(OCCU_RO_ARGS);
+#undef OCCU_RO_ARGS
   OCCU_PROF_END(ctx);
   LAUNCH_CHECK();
   return 1;

@@ -65,11 +65,20 @@ __device__ unsigned long long g_tc_time[32][4];
       g_tc_time[slot][0] += tt_w; g_tc_time[slot][1] += tt_b; g_tc_time[slot][2] += 1; \
     }                                                                             \
   } while (0)
+__device__ unsigned long long g_eg_time[32][4];
+#define TT_FLUSH_EG(slot)                                                         \
+  do {                                                                            \
+    tt_b += clock64() - tt_0;                                                     \
+    if (blockIdx.x == 0 && (threadIdx.x & 31) == 0) {                             \
+      g_eg_time[slot][0] += tt_w; g_eg_time[slot][1] += tt_b; g_eg_time[slot][2] += 1; \
+    }                                                                             \
+  } while (0)
 #else
 #define TT_DECL
 #define TT_WAIT_BEGIN
 #define TT_WAIT_END
 #define TT_FLUSH(slot)
+#define TT_FLUSH_EG(slot)
 #endif    // g = softmax(acc); m = g ⊙ h̄[s]; h[t] = LReLU(Σ_seg m) (a4-a6 fused)
 
 
@@ -243,6 +252,7 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
 
   // ---- weights: prebuilt fp16x2 images (wimage_kernel), bulk-copied by the producer ----
   const int fexp = __ldg(a.wfexp);
+  const bool noshift = __ldg(a.wfexp + 1) != 0;
   if (EPI == EPI_NODE)
     for (int i = threadIdx.x; i < D; i += NTH) {
       s.avec[i] = a.a_s[i];
@@ -686,18 +696,24 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
           }
         }
       } else if (EPI == EPI_GATE) {
-        float m = -INFINITY;
+        // g = softmax(logits) over channels; m = 0 when the weight bound allows (no max
+        // pass, see wimage_kernel), else the row max.
+        float m = 0.f;
+        if (!noshift) {
+          m = -INFINITY;
 #pragma unroll
-        for (int c0 = 0; c0 < DH; c0 += 16) {
-          uint32_t r[16];
-          tc::tmem_ld16(acc + c0, r);
-          tc::tmem_ld_wait();
+          for (int c0 = 0; c0 < DH; c0 += 16) {
+            uint32_t r[16];
+            tc::tmem_ld16(acc + c0, r);
+            tc::tmem_ld_wait();
 #pragma unroll
-          for (int u = 0; u < 16; ++u) m = fmaxf(m, __uint_as_float(r[u]) * un);
+            for (int u = 0; u < 16; ++u) m = fmaxf(m, __uint_as_float(r[u]) * un);
+          }
+          xg[hf * 128 + row] = m;
+          group_bar(g);
+          m = fmaxf(m, xg[(hf ^ 1) * 128 + row]);
         }
-        xg[hf * 128 + row] = m;
-        group_bar(g);
-        m = fmaxf(m, xg[(hf ^ 1) * 128 + row]);
+        const float unL = un * LOG2E, mL = m * LOG2E;
         float sum = 0.f;
 #pragma unroll
         for (int c0 = 0; c0 < DH; c0 += 16) {
@@ -705,13 +721,12 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
           tc::tmem_ld16(acc + c0, r);
           tc::tmem_ld_wait();
 #pragma unroll
-          for (int u = 0; u < 16; ++u) sum += fast_exp(__uint_as_float(r[u]) * un - m);
+          for (int u = 0; u < 16; ++u) sum += ex2(fmaf(__uint_as_float(r[u]), unL, -mL));
         }
         xg[256 + hf * 128 + row] = sum;
         group_bar(g);
         sum = hf == 0 ? sum + xg[256 + 128 + row] : xg[256 + row] + sum;   // fixed order
         const float inv = fast_rcp(sum);
-        const float unL = un * LOG2E, mL = m * LOG2E;
 #pragma unroll 1
         for (int c0 = 0; c0 < DH; c0 += 16) {
           uint32_t r[16];
@@ -781,6 +796,398 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
 }
 
 // ---------------------------------------------------------------------------
+// Fused edge transform + channel-softmax gate of one ANEE layer (a3 + a4, P145/P149):
+//   e' = σ(α · W_e e_in), α = p[s] + q[t];   g = softmax_c(W_m e')
+// e' is written once (next layer's input, kept for the backward) and never re-read
+// by the gate.  Persistent, one CTA per SM, 128-edge tiles, two chained tcgen05
+// GEMMs per tile (fp16x2-split operands, 3 products, FP32 accumulation in TMEM):
+//   warp 0       producer: TMA boxes (128 rows x 32 fp32) of e_in into a per-box ring
+//   warp 1       MMA: ACC1 = A1·W_eᵀ, ACC2 = A2·W_mᵀ (A from TMEM, B = weight images)
+//   warps 2-9    converters: e_in (in (0,1), unscaled) -> fp16x2 -> TMEM A1
+//   warps 10-17  stage 1: z = ACC1·2^-f_e, e' = σ(αz) -> HBM and fp16x2 -> TMEM A2
+//   warps 18-25  stage 2: softmax(ACC2·2^-f_m) -> HBM g
+// FIRST (layer 1, F_e <= 16): no A1 / MMA1; stage 1 forms z = W_e e0 on CUDA cores from
+// the raw edge_feat rows gathered through in_eid (a1 fused), writing e0_out if asked.
+// TMEM columns: A1 [0,128) ACC1 [128,256) A2 [256,384) ACC2 [384,512), single-buffered;
+// the MMA warp issues MMA1(i) before MMA2(i-1) so stage 1 never waits on stage 2.
+// ---------------------------------------------------------------------------
+struct EdgeGateArgs {
+  const float *e_in; int Ke, R;      // [R][Ke] (FIRST: raw edge_feat [R][Ke], row eid[k])
+  const int32_t *eid;                // FIRST: in-CSR edge -> edge_feat row
+  const float *W_e;                  // FIRST: [D][Ke] fp32 (CUDA-core path)
+  const uint8_t *wimg_e, *wimg_m;    // fp16x2 images [w0 | w1]
+  const int *wf_e, *wf_m;            // scale exponents (wf_m[1] = softmax no-shift flag)
+  const float *p, *q;
+  const int32_t *src, *dst;
+  float *e_out, *e0_out, *g;
+  int rev;
+  int dbg;                           // sensitivity experiments only (OCCU_EG_DBG), 0 in production
+};
+
+constexpr int EG_NTH = 832;
+
+__host__ __device__ inline size_t eg_smem_bytes(int D, int Ke, bool first) {
+  const size_t imgm = size_t(D) * D * 2;
+  const size_t imge = first ? size_t(Ke) * D * 4 / 2 : size_t(kpad_of(Ke)) * D * 2;  // 2 x imge total
+  const size_t ring = first ? 0 : size_t(nbox_of(Ke)) * 16384;
+  return 1024 + 2 * imgm + 2 * imge + ring + 256 + 2 * 2 * 128 * 4 + 16 * 16 * 20 * 4;
+}
+
+template <int D, int KM>      // KM > 0: FIRST (layer-1 CUDA-core edge transform, Ke <= KM)
+__global__ void __launch_bounds__(EG_NTH, 1) edgegate_kernel(const __grid_constant__ CUtensorMap tmap,
+                                                             EdgeGateArgs a) {
+  constexpr bool FIRST = KM > 0;
+  constexpr int KMX = FIRST ? KM : 1;
+  extern __shared__ uint8_t smem_raw[];
+  const int Ke = a.Ke, NB = FIRST ? 0 : nbox_of(Ke), Kpe = FIRST ? Ke : kpad_of(Ke);
+  uint8_t *base = smem_raw + ((1024 - (tc::smem_u32(smem_raw) & 1023)) & 1023);
+  const size_t imgm = size_t(D) * D * 2;
+  const size_t imge = FIRST ? size_t(Ke) * D * 4 / 2 : size_t(Kpe) * D * 2;
+  uint8_t *wm0 = base, *wm1 = base + imgm, *we0 = base + 2 * imgm, *we1 = we0 + imge;
+  float *ring = reinterpret_cast<float *>(we0 + 2 * imge);
+  uint8_t *misc = reinterpret_cast<uint8_t *>(ring) + (FIRST ? 0 : size_t(NB) * 16384);
+  uint64_t *bars = reinterpret_cast<uint64_t *>(misc);
+  uint64_t *full = bars, *empty = bars + 4, *a1full = bars + 8, *a1free = bars + 9,
+           *acc1full = bars + 10, *acc1free = bars + 11, *a2full = bars + 12, *a2free = bars + 13,
+           *acc2full = bars + 14, *acc2free = bars + 15, *wfull = bars + 16;
+  uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(misc + 160);
+  float *xg = reinterpret_cast<float *>(misc + 256);                 // stage 2: [2][2][128]
+  float *xbuf = xg + 2 * 2 * 128;                                    // 16 warps x 16 x 20
+  float *wt = reinterpret_cast<float *>(we0);                        // FIRST: W_eᵀ [Ke][D]
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+
+  if (FIRST)
+    for (int i = threadIdx.x; i < D * Ke; i += EG_NTH) wt[(i % Ke) * D + i / Ke] = a.W_e[i];
+  if (threadIdx.x == 0) {
+    for (int j = 0; j < 4; ++j) {
+      tc::mbar_init(full + j, 1);
+      tc::mbar_init(empty + j, 128);
+    }
+    tc::mbar_init(a1full, 256);
+    tc::mbar_init(a1free, 1);
+    tc::mbar_init(acc1full, 1);
+    tc::mbar_init(acc1free, 256);
+    tc::mbar_init(a2full, 256);
+    tc::mbar_init(a2free, 1);
+    tc::mbar_init(acc2full, 1);
+    tc::mbar_init(acc2free, 256);
+    tc::mbar_init(wfull, 1);
+    tc::fence_mbar_init();
+  }
+  if (warp == 1) tc::tmem_alloc<TMEM_COLS>(tmem_slot);
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+  tc::fence_before_sync();
+  __syncthreads();
+  tc::fence_after_sync();
+  const uint32_t tmem = *tmem_slot;
+  constexpr uint32_t A1 = 0, ACC1 = 128, A2 = 256, ACC2 = 384;
+  const int tiles = (a.R + TM - 1) / TM;
+  const int my = blockIdx.x < tiles ? (tiles - 1 - int(blockIdx.x)) / int(gridDim.x) + 1 : 0;
+  auto tile_r0 = [&](int i) -> long {
+    const int t = int(blockIdx.x) + i * int(gridDim.x);
+    return long(a.rev ? tiles - 1 - t : t) * TM;
+  };
+
+  if (warp == 0) {
+    if (lane == 0) {
+      if (!FIRST) tc::prefetch_tmap(&tmap);
+      const uint32_t bm = uint32_t(imgm), be = FIRST ? 0u : uint32_t(imge);
+      tc::mbar_arrive_expect_tx(wfull, 2 * bm + 2 * be);
+      for (uint32_t o = 0; o < bm; o += 16384) {
+        const uint32_t n = bm - o < 16384 ? bm - o : 16384;
+        tc::bulk_g2s(wm0 + o, a.wimg_m + o, n, wfull);
+        tc::bulk_g2s(wm1 + o, a.wimg_m + bm + o, n, wfull);
+      }
+      for (uint32_t o = 0; o < be; o += 16384) {
+        const uint32_t n = be - o < 16384 ? be - o : 16384;
+        tc::bulk_g2s(we0 + o, a.wimg_e + o, n, wfull);
+        tc::bulk_g2s(we1 + o, a.wimg_e + be + o, n, wfull);
+      }
+      TT_DECL
+      if (!FIRST)
+        for (int i = 0; i < my; ++i) {
+          const int r0 = int(tile_r0(i));
+          for (int b = 0; b < NB; ++b) {
+            TT_WAIT_BEGIN
+            if (i >= 1) tc::mbar_wait(empty + b, (i - 1) & 1);
+            TT_WAIT_END
+            tc::mbar_arrive_expect_tx(full + b, 16384u);
+            tc::tma_load_2d(ring + b * 4096, &tmap, 32 * b, r0, full + b);
+          }
+        }
+      TT_FLUSH_EG(0);
+    }
+    __syncwarp();
+  } else if (warp == 1) {
+    const uint32_t idsc = tc::idesc(128, uint32_t(D), tc::FMT_F16);
+    const uint32_t m0 = tc::smem_u32(wm0), m1 = tc::smem_u32(wm1);
+    const uint32_t e0a = tc::smem_u32(we0), e1a = tc::smem_u32(we1);
+    tc::mbar_wait(wfull, 0);
+    auto gemm = [&](uint32_t acc, uint32_t aop, uint32_t w0, uint32_t w1, int K, int Kp) {
+      for (int kk = 0; kk < K / 16; ++kk) {
+        const uint32_t boff = uint32_t(kk >> 2) * uint32_t(D) * 128u + uint32_t(kk & 3) * 32u;
+        const uint64_t b0 = tc::sdesc_sw128(w0 + boff), b1 = tc::sdesc_sw128(w1 + boff);
+        const uint32_t x0 = tmem + aop + uint32_t(kk) * 8u, x1 = x0 + uint32_t(Kp / 2);
+        tc::mma_f16_ts(tmem + acc, x0, b0, idsc, kk > 0 ? 1u : 0u);
+        tc::mma_f16_ts(tmem + acc, x0, b1, idsc, 1u);
+        tc::mma_f16_ts(tmem + acc, x1, b0, idsc, 1u);
+      }
+    };
+    TT_DECL
+    for (int i = 0; i <= my; ++i) {
+      if (!FIRST && i < my) {                    // MMA1(i)
+        TT_WAIT_BEGIN
+        tc::mbar_wait(a1full, i & 1);
+        if (i >= 1) tc::mbar_wait(acc1free, (i - 1) & 1);
+        TT_WAIT_END
+        tc::fence_after_sync();
+        if (lane == 0) {
+          gemm(ACC1, A1, e0a, e1a, Ke, Kpe);
+          tc::mma_commit(acc1full);
+          tc::mma_commit(a1free);
+        }
+        __syncwarp();
+      }
+      if (i >= 1) {                              // MMA2(i-1)
+        const int t = i - 1;
+        TT_WAIT_BEGIN
+        tc::mbar_wait(a2full, t & 1);
+        if (t >= 1) tc::mbar_wait(acc2free, (t - 1) & 1);
+        TT_WAIT_END
+        tc::fence_after_sync();
+        if (lane == 0) {
+          gemm(ACC2, A2, m0, m1, D, D);
+          tc::mma_commit(acc2full);
+          tc::mma_commit(a2free);
+        }
+        __syncwarp();
+      }
+    }
+    TT_FLUSH_EG(1);
+  } else if (warp < EPI0) {
+    if (!FIRST) {
+      // converters: thread = (row, K-half); e_in in (0,1) -> unscaled fp16x2 split
+      const int qd = warp & 3, kh = (warp - 2) >> 2, row = qd * 32 + lane;
+      const uint32_t lane_base = tmem + (uint32_t(qd * 32) << 16);
+      const int KH = Kpe / 2, kb = kh * KH, bpb = NB / 2;   // boxes per half
+      TT_DECL
+      for (int i = 0; i < my; ++i) {
+        const long r0 = tile_r0(i);
+        const bool live = row < min(TM, int(a.R - r0));
+        TT_WAIT_BEGIN
+        for (int b = 0; b < bpb; ++b) tc::mbar_wait(full + kh * bpb + b, i & 1);
+        if (i >= 1) tc::mbar_wait(a1free, (i - 1) & 1);
+        TT_WAIT_END
+        for (int c0 = 0; c0 < KH / 2; c0 += 16) {
+          uint32_t x0[16], x1[16];
+#pragma unroll
+          for (int u = 0; u < 16; u += 2) {
+            const int k = kb + 2 * (c0 + u);
+            float4 v = make_float4(0.f, 0.f, 0.f, 0.f);
+            if (live && k < Ke) v = slot_ld4(ring, row, k);
+            split2(v.x, v.y, x0[u], x1[u]);
+            split2(v.z, v.w, x0[u + 1], x1[u + 1]);
+          }
+          const uint32_t col = A1 + uint32_t(kb / 2 + c0);
+          tc::tmem_st16(lane_base + col, x0);
+          tc::tmem_st16(lane_base + col + Kpe / 2, x1);
+        }
+        tc::tmem_st_wait();
+        tc::fence_before_sync();
+        for (int b = 0; b < bpb; ++b) tc::mbar_arrive(empty + kh * bpb + b);
+        tc::mbar_arrive(a1full);
+      }
+      TT_FLUSH_EG(2 + (warp - 2));
+    }
+  } else if (warp < EPI0 + 8) {
+    // ---- stage 1: e' = σ(α z) -> HBM + fp16x2 -> A2 (thread = row, half hf of D) ----
+    const int wi = warp - EPI0, hf = wi >> 2, qd = warp & 3, row = qd * 32 + lane;
+    const uint32_t lane_base = tmem + (uint32_t(qd * 32) << 16);
+    float *wbuf = xbuf + wi * (16 * 20);
+    constexpr int DH = D / 2;
+    const int cb = hf * DH;
+    const float un = FIRST ? 1.f : ldexpf(1.f, -__ldg(a.wf_e));
+    // software-pipelined row inputs: indices of tile i+2 and values of tile i+1 are in
+    // flight while tile i is processed (α = p[s] + q[t] is a two-level gather)
+    auto rows_of = [&](int i, long &grow) {
+      const long r0 = tile_r0(i);
+      grow = r0 + row;
+      return i < my && row < min(TM, int(a.R - r0));
+    };
+    int s_n = 0, t_n = 0, x_n = 0;                   // indices of tile i+1
+    auto load_idx = [&](int i, int &sv, int &tv, int &xv) {
+      long gr;
+      if (rows_of(i, gr)) {
+        sv = __ldg(a.src + gr);
+        tv = __ldg(a.dst + gr);
+        if (FIRST) xv = a.eid ? __ldg(a.eid + gr) : int(gr);
+      }
+    };
+    float al_n = 0.f, ev_n[KMX];
+    auto load_val = [&](int i, int sv, int tv, int xv) {
+      long gr;
+      const bool lv = rows_of(i, gr);
+      al_n = lv ? __ldg(a.p + sv) + __ldg(a.q + tv) : 0.f;                     // α (R1)
+#pragma unroll
+      for (int j = 0; j < KMX; ++j)
+        ev_n[j] = (FIRST && lv && j < Ke) ? __ldg(a.e_in + long(xv) * Ke + j) : 0.f;
+    };
+    {
+      int s0 = 0, t0 = 0, x0 = 0;
+      load_idx(0, s0, t0, x0);
+      load_val(0, s0, t0, x0);
+      load_idx(1, s_n, t_n, x_n);
+    }
+    TT_DECL
+    for (int i = 0; i < my; ++i) {
+      const long r0 = tile_r0(i);
+      const int nrows = min(TM, int(a.R - r0));
+      const bool live = row < nrows;
+      const long grow = r0 + row;
+      const float al = al_n;
+      float ev[KMX];
+#pragma unroll
+      for (int j = 0; j < KMX; ++j) ev[j] = ev_n[j];
+      load_val(i + 1, s_n, t_n, x_n);                // tile i+1 values (indices ready)
+      load_idx(i + 2, s_n, t_n, x_n);                // tile i+2 indices
+      if (FIRST && a.e0_out && hf == 0 && live) {
+#pragma unroll
+        for (int j = 0; j < KMX; ++j)
+          if (j < Ke) a.e0_out[grow * Ke + j] = ev[j];
+      }
+      TT_WAIT_BEGIN
+      if (!FIRST) tc::mbar_wait(acc1full, i & 1);
+      if (i >= 1) tc::mbar_wait(a2free, (i - 1) & 1);
+      TT_WAIT_END
+      tc::fence_after_sync();
+      const float cexp = -al * un * LOG2E;
+      const long wrow0 = r0 + qd * 32;
+      const int wrows = max(0, min(32, nrows - qd * 32));
+#pragma unroll 1
+      for (int c0 = 0; c0 < DH; c0 += 16) {
+        float z[16];
+        if (FIRST) {
+#pragma unroll
+          for (int u = 0; u < 16; ++u) z[u] = 0.f;
+#pragma unroll
+          for (int j = 0; j < KMX; ++j) {
+            if (j >= Ke) break;
+            const float x = ev[j];
+#pragma unroll
+            for (int u = 0; u < 16; u += 4) {
+              const float4 w = *reinterpret_cast<const float4 *>(wt + j * D + cb + c0 + u);
+              z[u] = fmaf(w.x, x, z[u]); z[u + 1] = fmaf(w.y, x, z[u + 1]);
+              z[u + 2] = fmaf(w.z, x, z[u + 2]); z[u + 3] = fmaf(w.w, x, z[u + 3]);
+            }
+          }
+        } else {
+          uint32_t r[16];
+          tc::tmem_ld16(lane_base + ACC1 + cb + c0, r);
+          tc::tmem_ld_wait();
+#pragma unroll
+          for (int u = 0; u < 16; ++u) z[u] = __uint_as_float(r[u]);
+        }
+        float o[16];
+        if (a.dbg & 1) {
+#pragma unroll
+          for (int u = 0; u < 16; ++u) o[u] = fmaf(z[u], cexp, 0.5f);
+        } else {
+#pragma unroll
+          for (int u = 0; u < 16; ++u)                                        // e' (R2, R3)
+            o[u] = FIRST ? fast_rcp(1.f + fast_exp(-(al * z[u])))
+                         : fast_rcp(1.f + ex2(z[u] * cexp));
+        }
+        uint32_t x0[8], x1[8];
+#pragma unroll
+        for (int u = 0; u < 8; ++u) split2(o[2 * u], o[2 * u + 1], x0[u], x1[u]);
+        const uint32_t col = A2 + uint32_t((cb + c0) / 2);
+        tc::tmem_st8(lane_base + col, x0);
+        tc::tmem_st8(lane_base + col + D / 2, x1);
+        if (!(a.dbg & 4)) warp_store_chunk<D>(wbuf, a.e_out, wrow0, wrows, cb + c0, o, lane);
+      }
+      tc::tmem_st_wait();
+      tc::fence_before_sync();
+      if (!FIRST) tc::mbar_arrive(acc1free);
+      tc::mbar_arrive(a2full);
+    }
+    TT_FLUSH_EG(10 + wi);
+  } else {
+    // ---- stage 2: g = softmax(ACC2 · 2^-f_m) -> HBM ----
+    const int wi = warp - EPI0 - 8, hf = wi >> 2, qd = warp & 3, row = qd * 32 + lane;
+    const uint32_t lane_base = tmem + (uint32_t(qd * 32) << 16);
+    float *wbuf = xbuf + (8 + wi) * (16 * 20);
+    constexpr int DH = D / 2;
+    const int cb = hf * DH;
+    const float un = ldexpf(1.f, -__ldg(a.wf_m));
+    const bool noshift = __ldg(a.wf_m + 1) != 0;
+    TT_DECL
+    for (int i = 0; i < my; ++i) {
+      const long r0 = tile_r0(i);
+      const int nrows = min(TM, int(a.R - r0));
+      const long wrow0 = r0 + qd * 32;
+      const int wrows = max(0, min(32, nrows - qd * 32));
+      TT_WAIT_BEGIN
+      tc::mbar_wait(acc2full, i & 1);
+      TT_WAIT_END
+      tc::fence_after_sync();
+      const uint32_t acc = lane_base + ACC2 + cb;
+      float m = 0.f;
+      if (!noshift) {
+        m = -INFINITY;
+#pragma unroll
+        for (int c0 = 0; c0 < DH; c0 += 16) {
+          uint32_t r[16];
+          tc::tmem_ld16(acc + c0, r);
+          tc::tmem_ld_wait();
+#pragma unroll
+          for (int u = 0; u < 16; ++u) m = fmaxf(m, __uint_as_float(r[u]) * un);
+        }
+        xg[hf * 128 + row] = m;
+        group_bar(1);
+        m = fmaxf(m, xg[(hf ^ 1) * 128 + row]);
+      }
+      const float unL = un * LOG2E, mL = m * LOG2E;
+      float sum = 0.f;
+#pragma unroll
+      for (int c0 = 0; c0 < DH; c0 += 16) {
+        uint32_t r[16];
+        tc::tmem_ld16(acc + c0, r);
+        tc::tmem_ld_wait();
+#pragma unroll
+        for (int u = 0; u < 16; ++u) sum += ex2(fmaf(__uint_as_float(r[u]), unL, -mL));
+      }
+      xg[256 + hf * 128 + row] = sum;
+      group_bar(1);
+      sum = hf == 0 ? sum + xg[256 + 128 + row] : xg[256 + row] + sum;   // fixed order
+      const float inv = fast_rcp(sum);
+#pragma unroll 1
+      for (int c0 = 0; c0 < DH; c0 += 16) {
+        uint32_t r[16];
+        tc::tmem_ld16(acc + c0, r);
+        tc::tmem_ld_wait();
+        float o[16];
+        if (a.dbg & 8) {
+#pragma unroll
+          for (int u = 0; u < 16; ++u) o[u] = __uint_as_float(r[u]) * inv;
+        } else {
+#pragma unroll
+          for (int u = 0; u < 16; ++u) o[u] = ex2(fmaf(__uint_as_float(r[u]), unL, -mL)) * inv;
+        }
+        if (!(a.dbg & 2)) warp_store_chunk<D>(wbuf, a.g, wrow0, wrows, cb + c0, o, lane);
+      }
+      tc::fence_before_sync();
+      tc::mbar_arrive(acc2free);
+      group_bar(1);        // xg reused by the next tile
+    }
+    TT_FLUSH_EG(18 + wi);
+  }
+  tc::fence_before_sync();
+  __syncthreads();
+  tc::fence_after_sync();
+  if (warp == 1) tc::tmem_dealloc<TMEM_COLS>(tmem);
+}
+
+// ---------------------------------------------------------------------------
 // Weight images (built once per parameter update, shared by every row-GEMM launch):
 // scale exponent f (max |W|·2^f in [2^14, 2^15)), W·2^f split into fp16 hi / lo in the
 // SW128 K-major B-operand layout, [w0 | w1].  One CTA per matrix.
@@ -803,11 +1210,30 @@ __global__ void __launch_bounds__(256) wimage_kernel(const WImageJob *__restrict
   for (int o = 16; o > 0; o >>= 1) m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, o));
   if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = m;
   __syncthreads();
+  // largest row 1-norm of the matrix as used (rows n, columns k): a bound on |W x| for
+  // x in [0, 1]^K.  Gate logits W_m e' (e' in (0, 1)) then satisfy |logit| <= bound, and
+  // for bound <= 64 the channel softmax needs no max shift (exp cannot overflow or
+  // become subnormal; softmax is shift-invariant, so the result is the same function).
+  float rs = 0.f;
+  for (int n = threadIdx.x; n < D; n += 256) {
+    float a = 0.f;
+    for (int k = 0; k < K; ++k) a += fabsf(jb.transW ? jb.W[long(k) * D + n] : jb.W[long(n) * K + k]);
+    rs = fmaxf(rs, a);
+  }
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) rs = fmaxf(rs, __shfl_xor_sync(0xffffffffu, rs, o));
+  __shared__ float red2[8];
+  if ((threadIdx.x & 31) == 0) red2[threadIdx.x >> 5] = rs;
+  __syncthreads();
   if (threadIdx.x == 0) {
-    float mm = 0.f;
-    for (int w = 0; w < 8; ++w) mm = fmaxf(mm, red[w]);
+    float mm = 0.f, rr = 0.f;
+    for (int w = 0; w < 8; ++w) {
+      mm = fmaxf(mm, red[w]);
+      rr = fmaxf(rr, red2[w]);
+    }
     fe = scale_exp(mm);
-    *jb.fexp = fe;
+    jb.fexp[0] = fe;
+    jb.fexp[1] = rr <= 64.f ? 1 : 0;
   }
   __syncthreads();
   const float ws = ldexpf(1.f, fe);
@@ -1159,7 +1585,7 @@ const uint8_t *tc_wimg(const occu_ctx *ctx, int kind, int layer) {
   return ctx->wimg.as<uint8_t>() + size_t(layer * 6 + kind) * WIMG_MAX;
 }
 const int *tc_wfexp(const occu_ctx *ctx, int kind, int layer) {
-  return ctx->wfexp.as<int>() + layer * 6 + kind;
+  return ctx->wfexp.as<int>() + (layer * 6 + kind) * 2;     // [f, softmax no-shift flag]
 }
 
 // (Re)build the images when the parameters changed (set_params / Adam bump the version).
@@ -1168,7 +1594,7 @@ int tc_prepare_weights(occu_ctx *ctx, cudaStream_t st) {
   const occu_config &c = ctx->cfg;
   const ParamLayout &L = ctx->layout;
   if (ctx->wimg.ensure(size_t(c.L) * 6 * WIMG_MAX) != cudaSuccess ||
-      ctx->wfexp.ensure(size_t(c.L) * 6 * sizeof(int)) != cudaSuccess ||
+      ctx->wfexp.ensure(size_t(c.L) * 6 * 2 * sizeof(int)) != cudaSuccess ||
       ctx->wjobs.ensure(size_t(c.L) * 6 * sizeof(WImageJob)) != cudaSuccess)
     return -int(cudaErrorMemoryAllocation);
   std::vector<WImageJob> jobs;
@@ -1226,6 +1652,48 @@ static int launch_rowgemm(const occu_ctx *ctx, const RowGemmArgs &ra, const char
 }
 
 template <int D>
+static int launch_edgegate(const occu_ctx *ctx, const DevCsr &csr, int layer, const FwdLayerArgs &a,
+                           cudaStream_t st) {
+  if (csr.E <= 0) return 0;
+  const bool first = a.Ke <= 16;
+  EdgeGateArgs ea{};
+  ea.e_in = a.e_in; ea.Ke = a.Ke; ea.R = csr.E; ea.eid = a.e_eid; ea.W_e = a.W_e;
+  ea.wimg_m = tc_wimg(ctx, 2, layer); ea.wf_m = tc_wfexp(ctx, 2, layer);
+  if (!first) {
+    ea.wimg_e = tc_wimg(ctx, 1, layer);
+    ea.wf_e = tc_wfexp(ctx, 1, layer);
+  }
+  ea.p = a.p; ea.q = a.q; ea.src = csr.in_src; ea.dst = csr.in_dst;
+  ea.e_out = a.e_out; ea.e0_out = a.e0_out; ea.g = a.g;
+  ea.rev = ctx->l2_order;
+  static const int dbg = [] {
+    const char *e = getenv("OCCU_EG_DBG");
+    return e ? atoi(e) : 0;
+  }();
+  ea.dbg = dbg;
+  const size_t smem = eg_smem_bytes(D, a.Ke, first);
+  const int tiles = (csr.E + TM - 1) / TM;
+  const int grid = std::min(tiles, ctx->num_sms);
+  CUtensorMap tmap;
+  memset(&tmap, 0, sizeof(tmap));
+  if (!first && !encode_rows_map(&tmap, a.e_in, csr.E, a.Ke)) return -int(cudaErrorInvalidValue);
+  OCCU_PROF_BEGIN(ctx, "edge_gate_tc", st);
+  if (!first) {
+    set_smem(edgegate_kernel<D, 0>, smem);
+    edgegate_kernel<D, 0><<<grid, EG_NTH, smem, st>>>(tmap, ea);
+  } else if (a.Ke <= 4) {
+    set_smem(edgegate_kernel<D, 4>, smem);
+    edgegate_kernel<D, 4><<<grid, EG_NTH, smem, st>>>(tmap, ea);
+  } else {
+    set_smem(edgegate_kernel<D, 16>, smem);
+    edgegate_kernel<D, 16><<<grid, EG_NTH, smem, st>>>(tmap, ea);
+  }
+  OCCU_PROF_END(ctx);
+  TC_CHECK();
+  return 1;
+}
+
+template <int D>
 static int tc_forward_layer_impl(const occu_ctx *ctx, const DevCsr &csr, int layer,
                                  const FwdLayerArgs &a, float *partial, cudaStream_t st) {
   const float slope = ctx->cfg.slope;
@@ -1241,7 +1709,13 @@ static int tc_forward_layer_impl(const occu_ctx *ctx, const DevCsr &csr, int lay
   ra.rev = ctx->l2_order;
   if ((r = launch_rowgemm<D, EPI_NODE>(ctx, ra, "node_tc", st)) < 0) return r;
   n += r;
-  if (csr.E > 0) {
+  const bool fused_eg = ctx->path == 0 && ctx->fuse_edge_gate &&
+                        (a.Ke <= 16 || (a.Ke % 64 == 0 && a.Ke <= 128));
+  if (csr.E > 0 && fused_eg) {
+    // a3 + a4 fused: e' and g in one kernel (e' is not re-read)
+    if ((r = launch_edgegate<D>(ctx, csr, layer, a, st)) < 0) return r;
+    n += r;
+  } else if (csr.E > 0) {
     // a3: edge transform
     if (a.Ke <= 16) {
       const int grid = int(std::min<long>((long(csr.E) + 255) / 256, 8L * ctx->num_sms));
@@ -1378,6 +1852,13 @@ extern "C" int occu_debug_tc_time(unsigned long long *host) {
   cudaMemcpyFromSymbol(host, occu::g_tc_time, sizeof(occu::g_tc_time));
   static unsigned long long zero[32][4] = {};
   cudaMemcpyToSymbol(occu::g_tc_time, zero, sizeof(zero));
+  return 0;
+}
+extern "C" int occu_debug_eg_time(unsigned long long *host) {
+  cudaDeviceSynchronize();
+  cudaMemcpyFromSymbol(host, occu::g_eg_time, sizeof(occu::g_eg_time));
+  static unsigned long long zero[32][4] = {};
+  cudaMemcpyToSymbol(occu::g_eg_time, zero, sizeof(zero));
   return 0;
 }
 #endif

@@ -90,6 +90,7 @@ struct occu_ctx {
   bool keep = false;
   int path = 0;            // 0: tensor cores, 1: CUDA-core SIMT FP32, 2: tensor cores + fused aggregation
   int l2_order = 1;        // alternate row-walk direction between producer/consumer kernels (L2 reuse)
+  int fuse_edge_gate = 0;  // path 0: edge transform + gate in one kernel (edgegate_kernel), OCCU_FUSE_EG=1
   occu::DevBuf wimg, wjobs, wfexp;   // prebuilt tensor-core weight images (per parameter version)
   int64_t params_version = 0, wimg_version = -1;
   float weight_decay = 1e-4f;

@@ -10,7 +10,7 @@ def kname(full):
     if m:
         return ["node_tc", "edge_tc", "gate_tc", "plain_tc", "gatebwd_tc", "edgebwd_tc",
                 "gateagg_tc"][int(m.group(2))]
-    for k, v in [("edge_small", "edge_small"), ("wgrad_tc", "wgrad_tc"), ("wimage", "wimage"),
+    for k, v in [("edgegate", "edge_gate_tc"), ("edge_small", "edge_small"), ("wgrad_tc", "wgrad_tc"), ("wimage", "wimage"),
                  ("split_reduce", "split_reduce"), ("agg_fixup", "agg_fixup"),
                  ("wgrad_skinny", "wgrad_skinny"), ("gather_segsum", "gather_segsum"),
                  ("readout_head", "readout_head"), ("permute_rows", "permute_e0"),

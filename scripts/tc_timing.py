@@ -23,12 +23,17 @@ csr = m.to_device(occu.pack(b.graphs))
 nf = torch.from_numpy(b.node_feat).cuda(); ef = torch.from_numpy(b.edge_feat).cuda()
 L = occu.lib()
 buf = np.zeros((32, 4), np.uint64)
+ebuf = np.zeros((32, 4), np.uint64)
 m.predict(csr, nf, ef); torch.cuda.synchronize()
 L.occu_debug_tc_time(buf.ctypes.data_as(ctypes.c_void_p))   # reset
+L.occu_debug_eg_time(ebuf.ctypes.data_as(ctypes.c_void_p))
 m.predict(csr, nf, ef); torch.cuda.synchronize()
 L.occu_debug_tc_time(buf.ctypes.data_as(ctypes.c_void_p))
+L.occu_debug_eg_time(ebuf.ctypes.data_as(ctypes.c_void_p))
 names = ["producer", "mma"] + [f"conv{w}" for w in range(8)] + [f"epi{w}" for w in range(16)] + ["-", "-", "-", "-", "setup", "total"]
-for k, n in enumerate(names):
-    w, bsy, cnt = buf[k][0], buf[k][1], buf[k][2]
-    if cnt:
-        print(f"{n:9s} launches {cnt} wait {w/cnt:10.0f} busy {bsy/cnt:10.0f} cycles/launch")
+for title, b in (("rowgemm", buf), ("edgegate", ebuf)):
+    print("==", title)
+    for k, n in enumerate(names):
+        w, bsy, cnt = b[k][0], b[k][1], b[k][2]
+        if cnt:
+            print(f"{n:9s} launches {cnt} wait {w/cnt:10.0f} busy {bsy/cnt:10.0f} cycles/launch")

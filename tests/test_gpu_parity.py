@@ -221,7 +221,7 @@ def test_determinism_and_device_host_paths_bitwise():
     torch.cuda.synchronize()
     assert np.array_equal(y1, y2)
     assert np.array_equal(y1, y3.cpu().numpy())
-    assert m.last_launch_count() >= 3 * 3 + 2
+    assert m.last_launch_count() >= 3 * 3 + 1
 
 
 def test_batching_invariance_gpu():
