@@ -114,26 +114,28 @@ def readout_rows(graphs, chunk=8):
     return int(np.sum((off[1:] - 1) // chunk - off[:-1] // chunk + 1))
 
 
-def algorithmic_bytes(N, E, B, d=128, F_n=80, F_e=4, L=3, rrows=None):
-    """Per-step algorithmic bytes per kernel class (fp32 values, int32 indices).
-    rrows: readout partial rows when the readout is folded into the last aggregation
-    and the layer-1 edge kernel gathers edge_feat through in_eid (kernel path 0)."""
+def algorithmic_bytes(N, E, B, d=128, F_n=80, F_e=4, L=3, rrows=None, sa=4):
+    """Per-step algorithmic bytes per kernel class.  Inputs, p/q, α and readout partials are
+    FP32 (4 B), indices int32; sa = bytes per stored activation element (h̄, e', g, h):
+    4 (OCCU_FP32) or 2 (OCCU_BF16).  rrows: readout partial rows when the readout is folded
+    into the last aggregation and the layer-1 edge kernel gathers edge_feat through in_eid
+    (kernel path 0)."""
     s = 4
     fused = rrows is not None
-    node = s * N * F_n + s * N * d * (L - 1) + s * N * (d + 2) * L                # read h_in, write h̄,p,q
-    edge_small = s * E * F_e + 8 * E + 8 * N + s * E * d + (4 * E if fused else 0)  # layer 1
-    edge_tc = (L - 1) * (s * E * d + 8 * E + 8 * N + s * E * d)                    # layers 2..L
-    gate = L * (s * E * d + s * E * d)                                             # read e', write g
-    gather = L * (s * E * d + s * N * d + 4 * E + 4 * (N + 1))                     # g, h̄, idx
+    node = s * N * F_n + sa * N * d * (L - 1) + (sa * N * d + 8 * N) * L           # read h_in, write h̄,p,q
+    edge_small = s * E * F_e + 8 * E + 8 * N + sa * E * d + (4 * E if fused else 0)  # layer 1
+    edge_tc = (L - 1) * (sa * E * d + 8 * E + 8 * N + sa * E * d)                   # layers 2..L
+    gate = L * (sa * E * d + sa * E * d)                                            # read e', write g
+    gather = L * (sa * E * d + sa * N * d + 4 * E + 4 * (N + 1))                    # g, h̄, idx
     if fused:
-        gather += (L - 1) * s * N * d + 4 * N + s * rrows * d                      # h, node_graph, partials
+        gather += (L - 1) * sa * N * d + 4 * N + s * rrows * d                      # h, node_graph, partials
         readout = s * rrows * d + 4 * (B + 1) + s * B * (2 * d + 1)
     else:
-        gather += L * s * N * d
-        readout = s * N * d + s * B * (2 * d + 1)
+        gather += L * sa * N * d
+        readout = sa * N * d + s * B * (2 * d + 1)
     # fused edge transform + gate (edgegate_kernel): e' written once, never re-read
-    edge_gate = (s * E * F_e + 4 * E + 8 * E + 8 * N + 2 * s * E * d
-                 + (L - 1) * (s * E * d + 8 * E + 8 * N + 2 * s * E * d))
+    edge_gate = (s * E * F_e + 4 * E + 8 * E + 8 * N + 2 * sa * E * d
+                 + (L - 1) * (sa * E * d + 8 * E + 8 * N + 2 * sa * E * d))
     out = {"node_tc": node, "edge_small": edge_small, "edge_tc": edge_tc, "gate_tc": gate,
            "edge_gate_tc": edge_gate,
            "gather_segsum": gather, "readout_head": readout,
@@ -144,10 +146,10 @@ def algorithmic_bytes(N, E, B, d=128, F_n=80, F_e=4, L=3, rrows=None):
     return out
 
 
-def load_traffic():
+def load_traffic(name="traffic.json"):
     """Per-launch DRAM bytes (ncu dram__bytes_read+write) committed under profiles/."""
     try:
-        with open(os.path.join(ROOT, "profiles", "traffic.json")) as f:
+        with open(os.path.join(ROOT, "profiles", name)) as f:
             return json.load(f)
     except Exception:
         return {}
@@ -232,6 +234,7 @@ def main():
     ap.add_argument("--no-train", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--no-flush", action="store_true")
+    ap.add_argument("--no-bf16", action="store_true", help="skip the OCCU_BF16 inference line")
     ap.add_argument("--path", type=int, default=0, help="0: tcgen05 3xTF32 (default), 1: SIMT FP32")
     args = ap.parse_args()
     if args.warmup < 3:
@@ -272,13 +275,14 @@ def main():
     out = torch.empty(B, dtype=torch.float32, device=dev)
     flush = torch.empty(2 * L2_BYTES // 4, dtype=torch.float32, device=dev)
 
-    def timed(fn, steps, profile=False):
+    def timed(fn, steps, profile=False, mdl=None):
         """Per-step CUDA events on the launch stream; L2 flushed between steps."""
+        mdl = mdl or model
         ms = []
         launches = 0
         if profile:
-            model.profile_reset()
-            model.set_profiling(True)
+            mdl.profile_reset()
+            mdl.set_profiling(True)
         for _ in range(steps):
             if not args.no_flush:
                 flush.fill_(1.0)
@@ -287,11 +291,11 @@ def main():
             a.record(stream)
             fn()
             b.record(stream)
-            launches += model.last_launch_count()
+            launches += mdl.last_launch_count()
             ms.append((a, b))
         torch.cuda.synchronize()
         if profile:
-            model.set_profiling(False)
+            mdl.set_profiling(False)
         return [x.elapsed_time(y) for x, y in ms], launches
 
     def bar():
@@ -332,27 +336,33 @@ def main():
     # roofline: per-kernel device time inside the timed region (CUDA events on the
     # library's launch stream), algorithmic bytes per kernel
     d = 128
-    alg = algorithmic_bytes(N, E, B, d, rrows=readout_rows(batch.graphs) if args.path == 0 else None)
+    rrows = readout_rows(batch.graphs)
+    alg = algorithmic_bytes(N, E, B, d, rrows=rrows if args.path == 0 else None)
     traffic = load_traffic()
-    kernels = {}
-    for k, (ms_tot, n) in prof.items():
-        ms = ms_tot / args.steps
-        by = alg.get(k)
-        gbs = by / (ms * 1e-3) / 1e9 if (by and ms > 0) else None
-        kernels[k] = {"ms_per_step": ms, "launches_per_step": n / args.steps,
-                      "algorithmic_bytes_per_step": by, "achieved_GBps": gbs,
-                      "frac_of_measured_hbm": gbs / peaks["hbm_gbs"] if gbs else None}
-    dom = max(kernels, key=lambda k: kernels[k]["ms_per_step"])
-    tot_kernel = sum(v["ms_per_step"] for v in kernels.values())
-    kd = kernels[dom]
-    lpl = max(kd["launches_per_step"], 1)
-    tr = traffic.get(dom)
-    roof = {"kernel": dom, "bound": "hbm", "achieved": kd["achieved_GBps"], "peak": peaks["hbm_gbs"],
-            "unit": "GB/s", "frac": kd["frac_of_measured_hbm"],
-            "traffic": tr.get("dram_bytes_per_launch") if tr else None,
-            "algorithmic_bytes_per_launch": (kd["algorithmic_bytes_per_step"] or 0) / lpl,
-            "avg_launch_ms": kd["ms_per_step"] / lpl, "peak_kind": peak_src,
-            "share_of_step": kd["ms_per_step"] / tot_kernel if tot_kernel else None}
+
+    def kernel_table(prof, alg, traffic):
+        kernels = {}
+        for k, (ms_tot, n) in prof.items():
+            ms = ms_tot / args.steps
+            by = alg.get(k)
+            gbs = by / (ms * 1e-3) / 1e9 if (by and ms > 0) else None
+            kernels[k] = {"ms_per_step": ms, "launches_per_step": n / args.steps,
+                          "algorithmic_bytes_per_step": by, "achieved_GBps": gbs,
+                          "frac_of_measured_hbm": gbs / peaks["hbm_gbs"] if gbs else None}
+        dom = max(kernels, key=lambda k: kernels[k]["ms_per_step"])
+        tot_kernel = sum(v["ms_per_step"] for v in kernels.values())
+        kd = kernels[dom]
+        lpl = max(kd["launches_per_step"], 1)
+        tr = traffic.get(dom)
+        roof = {"kernel": dom, "bound": "hbm", "achieved": kd["achieved_GBps"], "peak": peaks["hbm_gbs"],
+                "unit": "GB/s", "frac": kd["frac_of_measured_hbm"],
+                "traffic": tr.get("dram_bytes_per_launch") if tr else None,
+                "algorithmic_bytes_per_launch": (kd["algorithmic_bytes_per_step"] or 0) / lpl,
+                "avg_launch_ms": kd["ms_per_step"] / lpl, "peak_kind": peak_src,
+                "share_of_step": kd["ms_per_step"] / tot_kernel if tot_kernel else None}
+        return kernels, roof
+
+    kernels, roof = kernel_table(prof, alg, traffic)
     agg_ms = kernels.get("gather_segsum", {}).get("ms_per_step")
     agg_launch = agg_ms / 3 if agg_ms else None
     agg_b = alg["gather_segsum"] / 3          # mean per launch over the L = 3 layers
@@ -364,6 +374,32 @@ def main():
     agg["frac_of_8TBps"] = agg["achieved"] / 8000.0 if agg["achieved"] else None
     if traffic.get("gather_segsum"):
         agg["traffic"] = traffic["gather_segsum"].get("dram_bytes_per_launch")
+
+    # ---- OCCU_BF16 inference on the same CFG2 batch (tolerance 1e-2; tests/test_gpu_bf16.py)
+    bf16 = None
+    if not args.no_bf16 and args.path == 0:
+        cb = occu.config(L=3, F_n=80, F_e=4, d=128, prec=occu.BF16)
+        mb = occu.Model(cb, device=local, stream=stream.cuda_stream)
+        mb.init_weights(42)
+        outb = torch.empty_like(out)
+        inferb = lambda: mb.predict(csr, nf, ef, outb)
+        with ClockSampler(local) as clkb:
+            timed(inferb, args.warmup, mdl=mb)
+            bar()
+            tb, lb = timed(inferb, args.steps, mdl=mb)
+            bar()
+            timed(inferb, args.steps, profile=True, mdl=mb)
+            bar()
+        msb = max_over_ranks(float(np.sum(tb)) / args.steps)
+        kb, roofb = kernel_table(mb.profile(), algorithmic_bytes(N, E, B, d, rrows=rrows, sa=2),
+                                 load_traffic("traffic_bf16.json"))
+        bf16 = {"value": B * world / (msb * 1e-3), "unit": "graphs/s", "ms_per_step": msb,
+                "dtype": "bf16", "tolerance": 1e-2, "gpu_launches": lb,
+                "precision": "OCCU_BF16: BF16 GEMM operands and stored activations (h̄, e', g, h), "
+                             "FP32 accumulation and everything else FP32",
+                "clocks": clkb.summary(), "roofline": roofb,
+                "kernel_ms_per_step": {k: v["ms_per_step"] for k, v in kb.items()}, "kernels": kb}
+        del mb
 
     # ---- e2e through the public API with host buffers (pinned), pack included
     pin_nf = torch.from_numpy(batch.node_feat).pin_memory()
@@ -437,6 +473,7 @@ def main():
                                      "over a second timed pass of the same K steps",
                               "ms_per_step_with_events": ms_step_prof},
             "e2e": e2e,
+            "bf16": bf16,
             "train": train,
             "cpu_baseline": cpu,
         }

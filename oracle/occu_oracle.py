@@ -218,6 +218,59 @@ def forward(params, cfg, pk, node_feat, edge_feat):
                 h0=np.asarray(node_feat, np.float64), r=r, c=c, o=o, yhat=yhat)
 
 
+# --------------------------------------------------------------------------
+# OCCU_BF16 mode (SURVEY §8(c) "Precision modes"; R24-R27): the same
+# forward with the BF16 roundings of the mode applied at the points where the
+# mode stores or feeds BF16, every operation itself in float64.  It defines what
+# the BF16 path computes up to FP32 summation order.
+# --------------------------------------------------------------------------
+def bf16_round(x):
+    """Round to the nearest bfloat16, ties to even (via float32, as FP32 -> BF16 RN)."""
+    b = np.ascontiguousarray(np.asarray(x, np.float64).astype(np.float32)).view(np.uint32)
+    b = (b + np.uint32(0x7FFF) + ((b >> np.uint32(16)) & np.uint32(1))) & np.uint32(0xFFFF0000)
+    return b.view(np.float32).astype(np.float64)
+
+
+def forward_bf16(params, cfg, pk, node_feat, edge_feat):
+    """Forward of OCCU_BF16: tensor-core GEMM operands (activations and W_u, W_e, W_m) are
+    rounded to BF16 (R24); stored h̄, e', g, h are BF16 (R24); p, q come from the unrounded
+    h̄ and, like α, σ, the softmax, the message product, the segment sums, the readout (over
+    the unrounded last-layer h, R27) and the head, stay unrounded.  The layer-1 edge
+    transform with F_e <= 16 is a CUDA-core FP32 step, not a tensor-core GEMM (R27)."""
+    r16 = bf16_round
+    slope = cfg["slope"]
+    s_k, t_k = pk["in_src"].astype(np.int64), pk["in_dst"].astype(np.int64)
+    N = pk["num_nodes"]
+    h = np.asarray(node_feat, np.float64)
+    e = np.asarray(edge_feat, np.float64)[pk["in_eid"].astype(np.int64)]
+    deg = np.diff(pk["in_ptr"].astype(np.int64))
+    layers = []
+    for i in range(cfg["L"]):
+        W_u, W_e, W_m = params[f"W_u{i}"], params[f"W_e{i}"], params[f"W_m{i}"]
+        P = r16(h) @ r16(W_u).T                                   # P141, BF16 operands
+        hbar_f = leaky_relu(P, slope)
+        p = hbar_f @ params[f"a_s{i}"]                            # P145/P147 (R1)
+        q = hbar_f @ params[f"a_d{i}"]
+        hbar = r16(hbar_f)                                        # stored BF16
+        alpha = p[s_k] + q[t_k]
+        tensor_core = not (i == 0 and e.shape[1] <= 16)
+        z = (r16(e) @ r16(W_e).T) if tensor_core else (e @ W_e.T)   # P145
+        e_new = r16(sigmoid(alpha[:, None] * z))                  # stored BF16
+        v = e_new @ r16(W_m).T                                    # P149
+        g = r16(softmax_channels(v))                              # stored BF16 (R24)
+        A = segment_sum(g * hbar[s_k], t_k, N)                    # P149 (R4, reading A)
+        if cfg["aggr"] == AGGR_MEAN:
+            A = A / np.maximum(deg, 1)[:, None]
+        h_f = leaky_relu(A, slope)
+        layers.append(dict(hbar=hbar, p=p, q=q, e=e_new, g=g, h=r16(h_f), h_f32=h_f))
+        h, e = r16(h_f), e_new
+    n_b = np.diff(pk["node_off"].astype(np.int64))
+    r = segment_sum(layers[-1]["h_f32"], pk["node_graph"].astype(np.int64), pk["num_graphs"]) / n_b[:, None]
+    c = r @ params["W_1"].T + params["b_1"]                       # P125 (R12)
+    yhat = leaky_relu(c, slope) @ params["w_2"] + params["b_2"][0]
+    return dict(layers=layers, r=r, c=c, yhat=yhat)
+
+
 def predict(params, cfg, graphs, node_feat, edge_feat):
     return forward(params, cfg, pack(graphs), node_feat, edge_feat)["yhat"]
 

@@ -11,6 +11,7 @@
 // Tiling: 64-row tiles, 256 threads as 16 (tx) x 16 (ty); thread owns rows
 // ty*4..ty*4+3 and columns {tx*4+j, 64+tx*4+j}.  The whole weight matrix sits
 // in shared memory (d <= 128), persistent CTAs loop over tiles.
+#include <cuda_bf16.h>
 #include <cuda_runtime.h>
 #include <math.h>
 #include <stdint.h>
@@ -393,11 +394,56 @@ __global__ void __launch_bounds__(NT) gather_segsum_kernel(
 // group issues G gathered (g, h̄[s]) row pairs unconditionally (indices clamped into
 // the chunk, surplus rows are never accumulated), and the next chunk's in_ptr /
 // in_src words are requested while the current chunk is summed.
-template <int D, int G, bool RP>
+template <int V, bool BF>
+__device__ __forceinline__ void load_row(const void *base, long row, int D, int lane, float (&v)[V]) {
+  if constexpr (BF) {
+    const __nv_bfloat16 *p = reinterpret_cast<const __nv_bfloat16 *>(base) + row * D + lane * V;
+    if constexpr (V == 4) {
+      const uint2 x = __ldg(reinterpret_cast<const uint2 *>(p));
+      const float2 a = __bfloat1622float2(*reinterpret_cast<const __nv_bfloat162 *>(&x.x));
+      const float2 b = __bfloat1622float2(*reinterpret_cast<const __nv_bfloat162 *>(&x.y));
+      v[0] = a.x; v[1 % V] = a.y; v[2 % V] = b.x; v[3 % V] = b.y;
+    } else {
+#pragma unroll
+      for (int c = 0; c < V; c += 2) {
+        const uint32_t x = __ldg(reinterpret_cast<const unsigned int *>(p + c));
+        const float2 a = __bfloat1622float2(*reinterpret_cast<const __nv_bfloat162 *>(&x));
+        v[c] = a.x; v[(c + 1) % V] = a.y;
+      }
+    }
+  } else {
+    const float *p = reinterpret_cast<const float *>(base) + row * D + lane * V;
+    if constexpr (V == 4) {
+      const float4 a = __ldg(reinterpret_cast<const float4 *>(p));
+      v[0] = a.x; v[1 % V] = a.y; v[2 % V] = a.z; v[3 % V] = a.w;
+    } else {
+#pragma unroll
+      for (int c = 0; c < V; ++c) v[c] = __ldg(p + c);
+    }
+  }
+}
+template <int V, bool BF>
+__device__ __forceinline__ void store_row_t(void *base, long row, int D, int lane, const float (&v)[V]) {
+  if constexpr (BF) {
+    __nv_bfloat16 *p = reinterpret_cast<__nv_bfloat16 *>(base) + row * D + lane * V;
+    uint32_t w[V / 2];
+#pragma unroll
+    for (int c = 0; c < V; c += 2) {
+      const __nv_bfloat162 h = __floats2bfloat162_rn(v[c], v[c + 1]);
+      w[c / 2] = *reinterpret_cast<const uint32_t *>(&h);
+    }
+    if constexpr (V == 4) *reinterpret_cast<uint2 *>(p) = make_uint2(w[0], w[1]);
+    else *reinterpret_cast<uint32_t *>(p) = w[0];
+  } else {
+    store_row<V>(reinterpret_cast<float *>(base) + row * D + lane * V, v);
+  }
+}
+
+template <int D, int G, bool RP, bool BF = false>
 __global__ void __launch_bounds__(NT, G == 4 ? 4 : 3) gather_segsum_v2_kernel(
-    const float *__restrict__ g, const float *__restrict__ hbar,
+    const void *__restrict__ g, const void *__restrict__ hbar,
     const int32_t *__restrict__ in_ptr, const int32_t *__restrict__ in_src, int N, int mean,
-    float slope, float *__restrict__ h_out, const int32_t *__restrict__ node_graph,
+    float slope, void *__restrict__ h_out, const int32_t *__restrict__ node_graph,
     float *__restrict__ rpart) {
   constexpr int V = D / 32;
   constexpr int NPW = 8;
@@ -439,7 +485,7 @@ __global__ void __launch_bounds__(NT, G == 4 ? 4 : 3) gather_segsum_v2_kernel(
         o[c] = lrelu(x, slope);
         acc[c] = 0.f;
       }
-      if (!RP || h_out) store_row<V>(h_out + (t0 + nd) * D + lane * V, o);
+      if (!RP || h_out) store_row_t<V, BF>(h_out, t0 + nd, D, lane, o);
       if (RP) {
         const int gc = __shfl_sync(0xffffffffu, gr_l, nd);
         const int gn = __shfl_sync(0xffffffffu, gr_l, (nd + 1) & 31);
@@ -464,20 +510,8 @@ __global__ void __launch_bounds__(NT, G == 4 ? 4 : 3) gather_segsum_v2_kernel(
         for (int u = 0; u < G; ++u) {
           const int kk = min(j + u, cnt - 1);
           const int sidx = __shfl_sync(0xffffffffu, s_l, kk);
-          const float *gr = g + long(base + kk) * D + lane * V;
-          const float *hr = hbar + long(sidx) * D + lane * V;
-          if constexpr (V == 4) {
-            const float4 a = __ldg(reinterpret_cast<const float4 *>(gr));
-            const float4 b = __ldg(reinterpret_cast<const float4 *>(hr));
-            gv[u][0] = a.x; gv[u][1 % V] = a.y; gv[u][2 % V] = a.z; gv[u][3 % V] = a.w;
-            hv[u][0] = b.x; hv[u][1 % V] = b.y; hv[u][2 % V] = b.z; hv[u][3 % V] = b.w;
-          } else {
-#pragma unroll
-            for (int c = 0; c < V; ++c) {
-              gv[u][c] = __ldg(gr + c);
-              hv[u][c] = __ldg(hr + c);
-            }
-          }
+          load_row<V, BF>(g, long(base + kk), D, lane, gv[u]);
+          load_row<V, BF>(hbar, long(sidx), D, lane, hv[u]);
         }
         if (!next_src_issued && t1 < N) {                      // next chunk's first sources
           const int nb = __shfl_sync(0xffffffffu, ptr_n, 0);
@@ -1183,6 +1217,33 @@ static int gather_impl(const occu_ctx *ctx, const DevCsr &csr, const float *g, c
   OCCU_PROF_END(ctx);
   LAUNCH_CHECK();
   return 1;
+}
+
+template <int D>
+static int gather_bf16_impl(const occu_ctx *ctx, const DevCsr &csr, const void *g, const void *hbar,
+                            void *h_out, float *rpart, cudaStream_t st) {
+  if (csr.N <= 0) return 0;
+  const int mean = ctx->cfg.aggr == OCCU_AGGR_MEAN;
+  const int grid = grid_for(long(csr.N) * 4, NT, 8 * ctx->num_sms);
+  OCCU_PROF_BEGIN(ctx, "gather_segsum", st);
+  if (rpart)
+    gather_segsum_v2_kernel<D, 4, true, true><<<grid, NT, 0, st>>>(
+        g, hbar, csr.in_ptr, csr.in_src, csr.N, mean, ctx->cfg.slope, h_out, csr.node_graph, rpart);
+  else
+    gather_segsum_v2_kernel<D, 4, false, true><<<grid, NT, 0, st>>>(
+        g, hbar, csr.in_ptr, csr.in_src, csr.N, mean, ctx->cfg.slope, h_out, csr.node_graph, rpart);
+  OCCU_PROF_END(ctx);
+  LAUNCH_CHECK();
+  return 1;
+}
+
+int launch_gather_segsum_bf16(const occu_ctx *ctx, const DevCsr &csr, const void *g,
+                              const void *hbar, void *h_out, float *rpart, cudaStream_t st) {
+  switch (ctx->cfg.d) {
+    case 64: return gather_bf16_impl<64>(ctx, csr, g, hbar, h_out, rpart, st);
+    case 128: return gather_bf16_impl<128>(ctx, csr, g, hbar, h_out, rpart, st);
+    default: return -int(cudaErrorInvalidValue);
+  }
 }
 
 int launch_gather_segsum(const occu_ctx *ctx, const DevCsr &csr, const float *g,

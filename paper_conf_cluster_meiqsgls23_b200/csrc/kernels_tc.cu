@@ -26,6 +26,7 @@
 //              the TMEM accumulator ACC[(i-1)%2] (tcgen05.ld).
 // TMEM: A[2] x 128 columns + ACC[2] x 128 columns = 512.  Loads of tile i+1,
 // the MMAs of tile i and the epilogue of tile i-1 overlap.
+#include <cuda_bf16.h>
 #include <cuda_fp16.h>
 #include <cuda_runtime.h>
 #include <math.h>
@@ -1197,6 +1198,7 @@ struct WImageJob {
   int D, K, transW;
   uint8_t *img;
   int *fexp;
+  int bf16;        // OCCU_BF16: one unscaled BF16 image (f = 0) instead of the fp16 pair
 };
 
 __global__ void __launch_bounds__(256) wimage_kernel(const WImageJob *__restrict__ jobs) {
@@ -1231,7 +1233,7 @@ __global__ void __launch_bounds__(256) wimage_kernel(const WImageJob *__restrict
       mm = fmaxf(mm, red[w]);
       rr = fmaxf(rr, red2[w]);
     }
-    fe = scale_exp(mm);
+    fe = jb.bf16 ? 0 : scale_exp(mm);
     jb.fexp[0] = fe;
     jb.fexp[1] = rr <= 64.f ? 1 : 0;
   }
@@ -1244,11 +1246,16 @@ __global__ void __launch_bounds__(256) wimage_kernel(const WImageJob *__restrict
     const long i1 = jb.transW ? long(k + 1) * D + n : long(n) * K + k + 1;
     const float v0 = k < K ? jb.W[i0] * ws : 0.f;
     const float v1 = k + 1 < K ? jb.W[i1] * ws : 0.f;
-    uint32_t hi, lo;
-    split2(v0, v1, hi, lo);
     const uint32_t off = tc::sw128_offset_f16(n, k, D);
-    *reinterpret_cast<uint32_t *>(jb.img + off) = hi;
-    *reinterpret_cast<uint32_t *>(jb.img + ib + off) = lo;
+    if (jb.bf16) {
+      const __nv_bfloat162 b = __floats2bfloat162_rn(v0, v1);
+      *reinterpret_cast<__nv_bfloat162 *>(jb.img + off) = b;
+    } else {
+      uint32_t hi, lo;
+      split2(v0, v1, hi, lo);
+      *reinterpret_cast<uint32_t *>(jb.img + off) = hi;
+      *reinterpret_cast<uint32_t *>(jb.img + ib + off) = lo;
+    }
   }
 }
 
@@ -1603,6 +1610,7 @@ int tc_prepare_weights(occu_ctx *ctx, cudaStream_t st) {
     auto add = [&](int kind, const float *W, int D, int K, int transW) {
       WImageJob j;
       j.W = W; j.D = D; j.K = K; j.transW = transW;
+      j.bf16 = c.prec == OCCU_BF16;
       j.img = const_cast<uint8_t *>(tc_wimg(ctx, kind, i));
       j.fexp = const_cast<int *>(tc_wfexp(ctx, kind, i));
       jobs.push_back(j);

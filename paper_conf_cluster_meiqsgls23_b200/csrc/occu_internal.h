@@ -151,6 +151,12 @@ int launch_forward_layer_tc(const occu_ctx *ctx, const DevCsr &csr, int layer, c
                             float *partial, cudaStream_t st);
 int launch_gather_segsum(const occu_ctx *ctx, const DevCsr &csr, const float *g,
                          const float *hbar, float *h_out, float *rpart, cudaStream_t st);
+// OCCU_BF16: g, h̄, h stored as BF16 (FP32 arithmetic); rpart stays FP32.
+int launch_gather_segsum_bf16(const occu_ctx *ctx, const DevCsr &csr, const void *g,
+                              const void *hbar, void *h_out, float *rpart, cudaStream_t st);
+// OCCU_BF16 forward layer (kernels_bf16.cu); FwdLayerArgs pointers to h̄, e', g, h hold BF16.
+int launch_forward_layer_bf16(const occu_ctx *ctx, const DevCsr &csr, int layer,
+                              const FwdLayerArgs &a, cudaStream_t st);
 int launch_permute_rows(const occu_ctx *ctx, const float *src, const int32_t *idx, int rows,
                         int width, float *dst, cudaStream_t st);
 // h: [N][d] last-layer states, or (chunked) the readout chunk partials of

@@ -155,7 +155,10 @@ occu_status validate_cfg(const occu_config *c) {
     return fail(nullptr, OCCU_EINVAL, "aggr must be SUM or MEAN");
   if (c->msg != OCCU_MSG_CHANNEL_SOFTMAX)
     return fail(nullptr, OCCU_EINVAL, "msg: only OCCU_MSG_CHANNEL_SOFTMAX (reading A) in this build");
-  if (c->prec != OCCU_FP32) return fail(nullptr, OCCU_EINVAL, "prec: only OCCU_FP32 in this build");
+  if (c->prec != OCCU_FP32 && c->prec != OCCU_BF16)
+    return fail(nullptr, OCCU_EINVAL, "prec must be OCCU_FP32 or OCCU_BF16");
+  if (c->prec == OCCU_BF16 && !(c->F_n <= 128 && (c->F_e <= 16 || c->F_e % 64 == 0)))
+    return fail(nullptr, OCCU_EINVAL, "OCCU_BF16 needs F_n <= 128 and F_e <= 16 or a multiple of 64");
   if (!(c->slope > 0.f && c->slope < 1.f)) return fail(nullptr, OCCU_EINVAL, "slope must be in (0,1)");
   return OCCU_OK;
 }
@@ -226,11 +229,12 @@ occu_status forward(occu_ctx *ctx, const DevCsr &csr, const float *nf, const flo
   if (st != OCCU_OK) return st;
   cudaStream_t s = ctx->stream;
   const float *P = ctx->params.as<float>();
-  const bool tc = ctx->path != 1 && tc_supported(c);
+  const bool bf = c.prec == OCCU_BF16;        // kernel path 0 only (occu_set_kernel_path)
+  const bool tc = bf || (ctx->path != 1 && tc_supported(c));
   // Tensor-core path fusions: a1's edge permutation folded into the layer-1 edge kernel,
   // and the readout's node sums folded into the last aggregation (chunk partials).
   const bool fuse_e0 = tc && c.F_e <= 16;
-  const bool fuse_ro = tc && ctx->path == 0;
+  const bool fuse_ro = tc && (bf || ctx->path == 0);
   if (!fuse_e0) LK(launch_permute_rows(ctx, ef, csr.in_eid, csr.E, c.F_e, w.e0.as<float>(), s), "permute e0");
   if (tc) LK(tc_prepare_weights(ctx, s), "weight images");
   float *rpart = nullptr;
@@ -262,6 +266,10 @@ occu_status forward(occu_ctx *ctx, const DevCsr &csr, const float *nf, const flo
       if (last && fuse_ro) {
         a.rpart = rpart;
         if (!save_all) a.h_out = nullptr;
+      }
+      if (bf) {
+        LK(launch_forward_layer_bf16(ctx, csr, i, a, s), "forward layer (bf16)");
+        continue;
       }
       CK(w.tcpart.ensure(tc_partial_floats(csr.E, c.d) * 4), "alloc tc partials");
       LK(launch_forward_layer_tc(ctx, csr, i, a, w.tcpart.as<float>(), s), "forward layer (tc)");
@@ -325,6 +333,8 @@ occu_status grads_impl(occu_ctx *ctx, const occu_batch *batch, const float *targ
   if (!batch || !batch->csr || !targets) return fail(ctx, OCCU_EINVAL, "batch/targets NULL");
   if (batch->global_num_graphs < batch->csr->num_graphs)
     return fail(ctx, OCCU_EINVAL, "global_num_graphs < local num_graphs");
+  if (ctx->cfg.prec == OCCU_BF16)
+    return fail(ctx, OCCU_EINVAL, "OCCU_BF16: training is not in this build (inference only)");
   ctx->launches = 0;
   if ((st = resolve_csr(ctx, batch->csr, csr)) != OCCU_OK) return st;
   if ((st = stage_inputs(ctx, csr, batch->node_feat, batch->edge_feat, targets, stg)) != OCCU_OK)
@@ -677,6 +687,8 @@ occu_status occu_set_kernel_path(occu_ctx *ctx, int path) {
   if (!ctx) return fail(nullptr, OCCU_EINVAL, "ctx is NULL");
   if (path < 0 || path > 2)
     return fail(ctx, OCCU_EINVAL, "path must be 0 (tensor cores), 1 (SIMT) or 2 (tensor cores, fused aggregation)");
+  if (ctx->cfg.prec == OCCU_BF16 && path != 0)
+    return fail(ctx, OCCU_EINVAL, "OCCU_BF16 runs on kernel path 0 only");
   ctx->path = path;
   return OCCU_OK;
 }
@@ -715,6 +727,16 @@ occu_status occu_get_tensor(occu_ctx *ctx, int32_t which, int32_t layer, void *h
   }
   if (bytes != need) return fail(ctx, OCCU_EINVAL, "byte count mismatch");
   CK(cudaSetDevice(ctx->device), "cudaSetDevice");
+  const bool widen = ctx->cfg.prec == OCCU_BF16 &&
+                     (which == OCCU_T_HBAR || which == OCCU_T_E || which == OCCU_T_H);
+  if (widen) {     // BF16 stores: copy the 16-bit words, widen to float32 (exact)
+    std::vector<uint16_t> tmp(need / 4);
+    CK(cudaMemcpyAsync(tmp.data(), src, need / 2, cudaMemcpyDeviceToHost, ctx->stream), "D2H");
+    CK(cudaStreamSynchronize(ctx->stream), "sync");
+    uint32_t *o = static_cast<uint32_t *>(host_dst);
+    for (size_t i = 0; i < tmp.size(); ++i) o[i] = uint32_t(tmp[i]) << 16;
+    return OCCU_OK;
+  }
   CK(cudaMemcpyAsync(host_dst, src, need, cudaMemcpyDeviceToHost, ctx->stream), "D2H");
   CK(cudaStreamSynchronize(ctx->stream), "sync");
   return OCCU_OK;

@@ -1,0 +1,176 @@
+"""GPU parity of the OCCU_BF16 inference path (SURVEY §8(c) "Precision modes"; north_star
+"≤1e-2 for the BF16 tensor-core path") against the float64 oracle.
+
+BF16 mode: GEMM operands and the stored activations h̄, e', h (and the gate scratch g,
+DESIGN.md R24) are BF16; every other step is FP32.  Intermediates are compared with the
+oracle's BF16-mode forward (oracle.forward_bf16, same roundings in float64) at 3e-3; the
+predictions with the float64 oracle at the mode's 1e-2: rel-L2 of the batch's ŷ vector, and per graph |ŷ - ŷ_ref| <= 1e-2 * max(|ŷ_ref|,
+0.1) — occupancy is a fraction in [0, 1], and near-zero predictions come from cancellation
+in the head, so the floor is 0.1 % occupancy (R25).  Closed-form special cases
+whose values are exactly representable in BF16 are checked bit-exactly.
+"""
+import numpy as np
+import pytest
+
+import oracle
+from occu_gen import configs, weights
+from paper_conf_cluster_meiqsgls23_b200 import occu
+
+pytestmark = pytest.mark.gpu
+TOL = 1e-2
+
+
+def mk(L, d, F_n=80, F_e=4, aggr=0):
+    return occu.config(L=L, F_n=F_n, F_e=F_e, d=d, aggr=aggr, prec=occu.BF16)
+
+
+def ocfg(c):
+    return dict(L=c.L, F_n=c.F_n, F_e=c.F_e, d=c.d, d_h=c.d_h, aggr=c.aggr, msg=c.msg,
+                slope=float(np.float32(c.slope)))
+
+
+def wcfg(c):
+    return weights.ModelConfig(L=c.L, F_n=c.F_n, F_e=c.F_e, d=c.d, d_h=c.d_h, aggr=c.aggr)
+
+
+def rel(a, b):
+    a = np.asarray(a, np.float64)
+    b = np.asarray(b, np.float64)
+    nb = np.linalg.norm(b)
+    return np.linalg.norm(a - b) / (nb if nb > 0 else 1.0)
+
+
+def check_y(y, yr):
+    y = np.asarray(y, np.float64)
+    assert rel(y, yr) <= TOL
+    assert np.all(np.abs(y - yr) <= TOL * np.maximum(np.abs(yr), 0.1)), np.abs(y - yr).max()
+
+
+def run(c, batch, flat, keep=True):
+    m = occu.Model(c)
+    m.set_params(flat)
+    m.keep_intermediates(keep)
+    y = m.predict(occu.pack(batch.graphs), batch.node_feat, batch.edge_feat)
+    params = oracle.unflatten(ocfg(c), flat.astype(np.float64))
+    pk = oracle.pack(batch.graphs)
+    ref = oracle.forward(params, ocfg(c), pk, batch.node_feat, batch.edge_feat)
+    return m, y, ref, pk
+
+
+TOL_EMU = 3e-3      # vs oracle.forward_bf16: FP32 summation order and BF16 rounding flips
+
+
+@pytest.mark.parametrize("wset", ["unit", "default"])
+@pytest.mark.parametrize("L,d,aggr,seed", [(2, 64, 0, 1), (3, 128, 0, 2), (3, 128, 1, 3),
+                                           (1, 64, 1, 4)])
+def test_bf16_random_batches_all_intermediates(L, d, aggr, seed, wset):
+    """Every intermediate vs the oracle's BF16-mode forward (oracle.forward_bf16: the same
+    roundings, float64 arithmetic; R24-R27) at 3e-3, and ŷ vs the float64
+    oracle at the mode's 1e-2."""
+    c = mk(L, d, aggr=aggr)
+    b = configs.random_dag_batch(40, 300 + seed, max_nodes=60, hub=True)
+    flat = weights.init_flat(wcfg(c), seed)
+    if wset == "unit":
+        flat = weights.unit_scale(wcfg(c), flat)
+    m, y, ref, pk = run(c, b, flat)
+    emu = oracle.forward_bf16(oracle.unflatten(ocfg(c), flat.astype(np.float64)), ocfg(c), pk,
+                              b.node_feat, b.edge_feat)
+    N, E, B = pk["num_nodes"], pk["num_edges"], pk["num_graphs"]
+    for i in range(L):
+        lay = emu["layers"][i]
+        assert rel(m.get_tensor(occu.T_HBAR, i, (N, d)), lay["hbar"]) <= TOL_EMU, ("hbar", i)
+        assert rel(m.get_tensor(occu.T_P, i, (N,)), lay["p"]) <= TOL_EMU, ("p", i)
+        assert rel(m.get_tensor(occu.T_Q, i, (N,)), lay["q"]) <= TOL_EMU, ("q", i)
+        assert rel(m.get_tensor(occu.T_E, i, (E, d)), lay["e"]) <= TOL_EMU, ("e", i)
+        assert rel(m.get_tensor(occu.T_H, i, (N, d)), lay["h"]) <= TOL_EMU, ("h", i)
+    assert rel(m.get_tensor(occu.T_R, 0, (B, d)), emu["r"]) <= TOL_EMU
+    assert rel(y, emu["yhat"]) <= TOL_EMU
+    check_y(y, ref["yhat"])
+
+
+def test_bf16_cfg2_subset_and_default_weights():
+    c = mk(3, 128)
+    b = configs.cfg2(12)
+    for flat in (weights.unit_scale(wcfg(c), weights.init_flat(wcfg(c), 42)),
+                 weights.init_flat(wcfg(c), 42)):
+        m, y, ref, pk = run(c, b, flat, keep=False)
+        assert rel(m.get_tensor(occu.T_R, 0, (pk["num_graphs"], c.d)), ref["r"]) <= TOL
+        check_y(y, ref["yhat"])
+
+
+def test_bf16_cfg2_full_size_sampled_graphs():
+    """CFG2 at full size on device buffers, as bench.py runs the BF16 line; 6 sampled
+    graphs checked against the oracle one by one."""
+    import torch
+    c = mk(3, 128)
+    b = configs.cfg2(256)
+    flat = weights.unit_scale(wcfg(c), weights.init_flat(wcfg(c), 42))
+    m = occu.Model(c)
+    m.set_params(flat)
+    csr = m.to_device(occu.pack(b.graphs))
+    y = m.predict(csr, torch.from_numpy(b.node_feat).cuda(), torch.from_numpy(b.edge_feat).cuda())
+    torch.cuda.synchronize()
+    y = y.cpu().numpy()
+    params = oracle.unflatten(ocfg(c), flat.astype(np.float64))
+    for gi in (0, 1, 77, 128, 200, 255):
+        s = b.subset([gi])
+        yr = oracle.predict(params, ocfg(c), s.graphs, s.node_feat, s.edge_feat)
+        assert abs(y[gi] - yr[0]) <= TOL * max(abs(yr[0]), 0.1), gi
+
+
+def test_bf16_path_counts_exact():
+    """W_u = I, a = 0, W_m = 0, SUM, small integer X: h^i = (Aᵀ)^i X / d^i with integer
+    path counts < 256 — every stored value is exactly representable in BF16, so the BF16
+    path is bit-exact; e' ≡ 1/2."""
+    d = 64
+    c = mk(3, d, F_n=d, F_e=4)
+    b = configs.random_dag_batch(20, 77, max_nodes=30, f_n=d, hub=False)
+    X = np.floor(b.node_feat * 4).astype(np.float32)
+    p = weights.unflatten(wcfg(c), weights.init_flat(wcfg(c), 5).copy())
+    for i in range(3):
+        p[f"W_u{i}"] = np.eye(d, dtype=np.float32)
+        p[f"a_s{i}"][:] = 0
+        p[f"a_d{i}"][:] = 0
+        p[f"W_m{i}"][:] = 0
+    m = occu.Model(c)
+    m.set_params(weights.flatten(wcfg(c), p))
+    m.keep_intermediates(True)
+    m.predict(occu.pack(b.graphs), X, b.edge_feat)
+    pk = oracle.pack(b.graphs)
+    N = pk["num_nodes"]
+    adj = np.zeros((N, N), np.float64)
+    for s, t in zip(pk["in_src"], pk["in_dst"]):
+        adj[s, t] += 1
+    H = X.astype(np.float64)
+    for i in range(3):
+        H = adj.T @ H / d
+        assert np.max(H * d ** (i + 1)) < 256
+        assert np.array_equal(m.get_tensor(occu.T_H, i, (N, d)).astype(np.float64), H), i
+        assert np.all(m.get_tensor(occu.T_E, i, (pk["num_edges"], d)) == 0.5)
+
+
+def test_bf16_batching_and_determinism():
+    c = mk(3, 128)
+    b = configs.random_dag_batch(24, 91, max_nodes=50, hub=True)
+    flat = weights.unit_scale(wcfg(c), weights.init_flat(wcfg(c), 3))
+    m = occu.Model(c)
+    m.set_params(flat)
+    csr = occu.pack(b.graphs)
+    y1 = m.predict(csr, b.node_feat, b.edge_feat)
+    y2 = m.predict(csr, b.node_feat, b.edge_feat)
+    assert np.array_equal(y1, y2)
+    for gi in (0, 5, 23):
+        s = b.subset([gi])
+        ys = m.predict(occu.pack(s.graphs), s.node_feat, s.edge_feat)
+        assert abs(ys[0] - y1[gi]) <= TOL * max(abs(y1[gi]), 0.1)
+
+
+def test_bf16_errors():
+    c = mk(2, 64)
+    m = occu.Model(c)
+    m.init_weights(1)
+    with pytest.raises(occu.OccuError):
+        m.set_kernel_path(1)
+    b = configs.random_dag_batch(4, 5, max_nodes=10)
+    with pytest.raises(occu.OccuError):
+        m.train_step(occu.pack(b.graphs), b.node_feat, b.edge_feat, b.targets, 1e-4)

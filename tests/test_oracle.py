@@ -404,3 +404,59 @@ def test_adam_matches_torch_optim():
         opt.step()
         p, st = oracle.adam_step(p, {"w": g}, st, 1e-3, 1e-4)
     assert np.allclose(p["w"], tw.detach().numpy(), rtol=1e-12, atol=1e-15)
+
+
+# ------------------------------------------------ OCCU_BF16 emulation (R24-R27)
+def test_bf16_round_ties_and_library():
+    """bf16_round = round-to-nearest-even to 8 significant bits: hand-worked ties and
+    torch's own float32 -> bfloat16 conversion (an independent library routine)."""
+    import torch
+    r = oracle.bf16_round
+    assert r(1.0) == 1.0
+    assert r(1 + 2 ** -8) == 1.0                        # tie -> even mantissa (1.0)
+    assert r(1 + 3 * 2 ** -8) == 1 + 2 ** -6            # tie between 1+2^-7 (odd) and 1+2^-6
+    assert r(1 + 2 ** -8 + 2 ** -20) == 1 + 2 ** -7     # above the tie
+    assert r(-(1 + 3 * 2 ** -8)) == -(1 + 2 ** -6)
+    assert r(0.0) == 0.0 and r(2.0 ** 100) == 2.0 ** 100
+    x = np.random.default_rng(5).standard_normal(10000) * np.exp(np.random.default_rng(6).uniform(-20, 20, 10000))
+    ref = torch.tensor(x, dtype=torch.float32).to(torch.bfloat16).to(torch.float64).numpy()
+    assert np.array_equal(r(x), ref)
+
+
+def test_forward_bf16_equals_forward_when_rounding_is_exact():
+    """T3-style inputs (integers, W_u = I, a = 0, W_m = 0) make every BF16 rounding an
+    identity (e' = 1/2, g = 1/d, small dyadic h), so the BF16 forward equals the plain one."""
+    d = 4
+    cfg = cfg_dict(L=2, F_n=d, F_e=d, d=d, d_h=d)
+    graphs = [(4, np.array([0, 0, 1, 2], np.int32), np.array([1, 2, 3, 3], np.int32))]
+    X = np.array([[1, 2, 3, 0], [0, 1, 0, 0], [2, 0, 0, 1], [0, 0, 0, 0]], np.float64)
+    EF = np.random.default_rng(1).uniform(size=(4, d))
+    p = toy_params(cfg, W_u0=np.eye(d), W_u1=np.eye(d), W_e0=np.ones((d, d)), W_e1=np.ones((d, d)),
+                   W_1=np.eye(d), w_2=np.ones(d))
+    pk = oracle.pack(graphs)
+    a = oracle.forward(p, cfg, pk, X, EF)
+    b = oracle.forward_bf16(p, cfg, pk, X, EF)
+    for i in range(2):
+        for k in ("hbar", "p", "q", "e", "g", "h"):
+            assert np.array_equal(a["layers"][i][k], b["layers"][i][k]), (i, k)
+    assert np.array_equal(a["yhat"], b["yhat"])
+
+
+def test_forward_bf16_rounds_where_the_mode_says():
+    """Random weights: stored h̄, e', g, h are BF16 values; p is computed from the
+    unrounded h̄ (so it differs from h̄_bf16·a_s); the whole stays within the BF16 budget."""
+    cfg = cfg_dict(L=2, F_n=80, F_e=4, d=16, d_h=16)
+    b = configs.random_dag_batch(6, 44, max_nodes=20)
+    flat = weights.init_flat(weights.ModelConfig(L=2, d=16, d_h=16), 9)
+    p = oracle.unflatten(cfg, flat.astype(np.float64))
+    pk = oracle.pack(b.graphs)
+    f = oracle.forward_bf16(p, cfg, pk, b.node_feat, b.edge_feat)
+    g = oracle.forward(p, cfg, pk, b.node_feat, b.edge_feat)
+    for i in range(2):
+        lay = f["layers"][i]
+        for k in ("hbar", "e", "g", "h"):
+            assert np.array_equal(oracle.bf16_round(lay[k]), lay[k]), (i, k)
+        assert not np.array_equal(lay["p"], lay["hbar"] @ p[f"a_s{i}"])
+        for k in ("hbar", "p", "e", "h"):
+            ref = g["layers"][i][k]
+            assert np.linalg.norm(lay[k] - ref) <= 2e-2 * np.linalg.norm(ref), (i, k)
