@@ -75,7 +75,7 @@ __host__ __device__ inline int ring_slots(bool af32) { return af32 ? 2 : 4; }
 constexpr int XB_WORDS = 32 * 12;   // per-warp transpose buffer: 32 rows x (8 + 4 pad) words
 __host__ __device__ inline size_t bf_smem_bytes(int D, int K, bool af32) {
   return 1024 + size_t(kpad64(K)) * D * 2 + size_t(ring_slots(af32)) * slot_bytes(K, af32) + 512 +
-         2 * 2 * 2 * 128 * 4 + 2 * D * 4 + 16 * XB_WORDS * 4;
+         3 * 2 * 2 * 128 * 4 + 2 * D * 4 + 24 * XB_WORDS * 4;
 }
 
 // Coalesced BF16 store of a 16-column chunk of the warp's 32 rows (thread = row):
@@ -115,18 +115,13 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_bf16_kernel(const __grid_const
   uint8_t *misc = ring + size_t(NS) * SB;
   uint64_t *bars = reinterpret_cast<uint64_t *>(misc);
   uint64_t *full = bars, *empty = bars + 4, *afull = bars + 8, *afree = bars + 10,
-           *accfull = bars + 12, *accfree = bars + 14, *wfull = bars + 16;
+           *accfull = bars + 12, *accfree = bars + 15, *wfull = bars + 18;
   uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(misc + 256);
-  float *xch = reinterpret_cast<float *>(misc + 512);              // [2 groups][2][2][128]
-  float *avec = xch + 2 * 2 * 2 * 128;                             // [2*D]
-  uint32_t *xbuf = reinterpret_cast<uint32_t *>(avec + 2 * D);     // 16 x XB_WORDS
+  float *xch = reinterpret_cast<float *>(misc + 512);              // [3 groups][2][2][128]
+  float *avec = xch + 3 * 2 * 2 * 128;                             // [2*D]
+  uint32_t *xbuf = reinterpret_cast<uint32_t *>(avec + 2 * D);     // 24 x XB_WORDS
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-
-  if (EPI == EPI_NODE)
-    for (int i = threadIdx.x; i < D; i += NTH) {
-      avec[i] = a.a_s[i];
-      avec[D + i] = a.a_d[i];
-    }
+  pdl_trigger();
   if (threadIdx.x == 0) {
     for (int j = 0; j < 4; ++j) {
       tc::mbar_init(full + j, 1);
@@ -135,6 +130,8 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_bf16_kernel(const __grid_const
     for (int j = 0; j < 2; ++j) {
       tc::mbar_init(afull + j, 256);
       tc::mbar_init(afree + j, 1);
+    }
+    for (int j = 0; j < 3; ++j) {
       tc::mbar_init(accfull + j, 1);
       tc::mbar_init(accfree + j, 256);
     }
@@ -142,6 +139,12 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_bf16_kernel(const __grid_const
     tc::fence_mbar_init();
   }
   if (warp == 1) tc::tmem_alloc<512>(tmem_slot);
+  pdl_wait();                              // predecessor's writes visible from here on
+  if (EPI == EPI_NODE)
+    for (int i = threadIdx.x; i < D; i += NTH) {
+      avec[i] = a.a_s[i];
+      avec[D + i] = a.a_d[i];
+    }
   tc::fence_before_sync();
   __syncthreads();
   tc::fence_after_sync();
@@ -153,7 +156,12 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_bf16_kernel(const __grid_const
     return long(a.rev ? tiles - 1 - t : t) * TM;
   };
   auto a_col = [](int j) { return uint32_t(j) * 128u; };
-  auto acc_col = [](int j) { return 256u + uint32_t(j) * 128u; };
+  // BF16 input: no TMEM A operand and no converters, so the converter warps form a third
+  // epilogue group and three accumulators rotate (cols 0/128/256); FP32 input: A[2] at
+  // cols 0/128, two accumulators at 256/384, two epilogue groups.
+  constexpr int NG = AF32 ? 2 : 3;
+  constexpr int EW0 = AF32 ? EPI0 : 2;
+  auto acc_col = [](int j) { return (AF32 ? 256u : 0u) + uint32_t(j) * 128u; };
 
   if (warp == 0) {
     if (lane == 0) {
@@ -179,13 +187,13 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_bf16_kernel(const __grid_const
     const int nk = Kp / 16;
     tc::mbar_wait(wfull, 0);
     for (int i = 0; i < my; ++i) {
-      const int j = i & 1, s = i % NS;
+      const int j = i & 1, s = i % NS, ja = i % NG;
       if (AF32) tc::mbar_wait(afull + j, (i >> 1) & 1);
       else tc::mbar_wait(full + s, (i / NS) & 1);
-      if (i >= 2) tc::mbar_wait(accfree + j, ((i >> 1) - 1) & 1);
+      if (i >= NG) tc::mbar_wait(accfree + ja, ((i / NG) - 1) & 1);
       tc::fence_after_sync();
       if (lane == 0) {
-        const uint32_t d = tmem + acc_col(j);
+        const uint32_t d = tmem + acc_col(ja);
         for (int kk = 0; kk < nk; ++kk) {
           const uint32_t boff = uint32_t(kk >> 2) * uint32_t(D) * 128u + uint32_t(kk & 3) * 32u;
           const uint64_t bdesc = tc::sdesc_sw128(wa + boff);
@@ -196,14 +204,14 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_bf16_kernel(const __grid_const
             tc::mma_f16_ss(d, tc::sdesc_sw128(ra + aoff), bdesc, idsc, kk > 0 ? 1u : 0u);
           }
         }
-        tc::mma_commit(accfull + j);
+        tc::mma_commit(accfull + ja);
         if (AF32) tc::mma_commit(afree + j);
         else tc::mma_commit(empty + s);
       }
       __syncwarp();
     }
-  } else if (warp < EPI0) {
-    if (AF32) {
+  } else if (warp < EW0) {
+    {
       // converters: thread = (row, K-half), FP32 -> BF16 pairs -> TMEM A[j]
       const int qd = warp & 3, kh = (warp - 2) >> 2, row = qd * 32 + lane;
       const uint32_t lane_base = tmem + (uint32_t(qd * 32) << 16);
@@ -238,7 +246,7 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_bf16_kernel(const __grid_const
     }
   } else {
     // ---------------- epilogue: two groups of 8 warps on alternating tiles ----------------
-    const int wi = warp - EPI0, g = wi >> 3, hf = (wi >> 2) & 1, qd = warp & 3;
+    const int wi = warp - EW0, g = wi >> 3, hf = (wi >> 2) & 1, qd = warp & 3;
     const int row = qd * 32 + lane;
     const uint32_t lane_base = tmem + (uint32_t(qd * 32) << 16);
     float *xg = xch + g * (2 * 2 * 128);
@@ -246,8 +254,8 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_bf16_kernel(const __grid_const
     constexpr int DH = D / 2;
     const int cb = hf * DH;
     const bool noshift = EPI == EPI_GATE && __ldg(a.wf + 1) != 0;
-    for (int i = g; i < my; i += 2) {
-      const int j = i & 1;
+    for (int i = g; i < my; i += NG) {
+      const int j = i % NG;
       const long r0 = tile_r0(i);
       const int nrows = min(TM, int(a.R - r0));
       const bool live = row < nrows;
@@ -256,7 +264,7 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_bf16_kernel(const __grid_const
       const int wrows = max(0, min(32, nrows - qd * 32));
       float al = 0.f;
       if (EPI == EPI_EDGE && live) al = __ldg(a.pin + __ldg(a.src + grow)) + __ldg(a.qin + __ldg(a.dst + grow));
-      tc::mbar_wait(accfull + j, (i >> 1) & 1);
+      tc::mbar_wait(accfull + j, (i / NG) & 1);
       tc::fence_after_sync();
       const uint32_t acc = lane_base + acc_col(j) + cb;
       if (EPI == EPI_NODE) {
@@ -356,6 +364,8 @@ __global__ void __launch_bounds__(256) edge_small_bf16_kernel(
     __nv_bfloat16 *__restrict__ e_out, float *__restrict__ e0_out) {
   constexpr int V = D / 32;
   extern __shared__ float wsm[];
+  pdl_trigger();
+  pdl_wait();
   for (int i = threadIdx.x; i < D * Ke; i += blockDim.x) wsm[(i % Ke) * D + i / Ke] = W_e[i];
   __syncthreads();
   const int lane = threadIdx.x & 31;
@@ -446,7 +456,7 @@ int launch_bf(const occu_ctx *ctx, const BfArgs &ra, const void *A, const char *
   CUtensorMap tmap;
   if (!encode_map(&tmap, A, ra.R, ra.K, !AF32)) return -int(cudaErrorInvalidValue);
   OCCU_PROF_BEGIN(ctx, name, st);
-  rowgemm_bf16_kernel<D, EPI, AF32><<<grid, NTH, smem, st>>>(tmap, ra);
+  launch_pdl(ctx->pdl & 16, rowgemm_bf16_kernel<D, EPI, AF32>, grid, NTH, smem, st, tmap, ra);
   OCCU_PROF_END(ctx);
   const cudaError_t e = cudaGetLastError();
   return e == cudaSuccess ? 1 : -int(e);
@@ -474,11 +484,11 @@ int forward_layer_bf16(const occu_ctx *ctx, const DevCsr &csr, int layer, const 
       const int grid = int(std::min<long>((long(csr.E) + 255) / 256, 8L * ctx->num_sms));
       OCCU_PROF_BEGIN(ctx, "edge_small", st);
       if (a.Ke <= 4)
-        edge_small_bf16_kernel<D, 4><<<grid, 256, D * a.Ke * 4, st>>>(
-            a.e_in, a.Ke, a.W_e, a.p, a.q, csr.in_src, csr.in_dst, a.e_eid, csr.E, e_out, a.e0_out);
+        launch_pdl(ctx->pdl & 4, edge_small_bf16_kernel<D, 4>, grid, 256, D * a.Ke * 4, st, a.e_in, a.Ke,
+                   a.W_e, a.p, a.q, csr.in_src, csr.in_dst, a.e_eid, csr.E, e_out, a.e0_out);
       else
-        edge_small_bf16_kernel<D, 16><<<grid, 256, D * a.Ke * 4, st>>>(
-            a.e_in, a.Ke, a.W_e, a.p, a.q, csr.in_src, csr.in_dst, a.e_eid, csr.E, e_out, a.e0_out);
+        launch_pdl(ctx->pdl & 4, edge_small_bf16_kernel<D, 16>, grid, 256, D * a.Ke * 4, st, a.e_in, a.Ke,
+                   a.W_e, a.p, a.q, csr.in_src, csr.in_dst, a.e_eid, csr.E, e_out, a.e0_out);
       OCCU_PROF_END(ctx);
       const cudaError_t e = cudaGetLastError();
       if (e != cudaSuccess) return -int(e);

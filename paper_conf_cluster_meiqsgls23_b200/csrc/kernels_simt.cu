@@ -422,6 +422,43 @@ __device__ __forceinline__ void load_row(const void *base, long row, int D, int 
     }
   }
 }
+// A lane's V-channel slice of a stored row, kept in its storage type until use (BF16
+// rows stay packed: half the registers per row in flight).
+template <int V, bool BF> struct RawRow;
+template <> struct RawRow<4, false> {
+  float4 v;
+  __device__ __forceinline__ void load(const void *b, long row, int D, int lane) {
+    v = __ldg(reinterpret_cast<const float4 *>(reinterpret_cast<const float *>(b) + row * D + lane * 4));
+  }
+  __device__ __forceinline__ void get(float (&o)[4]) const { o[0] = v.x; o[1] = v.y; o[2] = v.z; o[3] = v.w; }
+};
+template <> struct RawRow<2, false> {
+  float2 v;
+  __device__ __forceinline__ void load(const void *b, long row, int D, int lane) {
+    v = __ldg(reinterpret_cast<const float2 *>(reinterpret_cast<const float *>(b) + row * D + lane * 2));
+  }
+  __device__ __forceinline__ void get(float (&o)[2]) const { o[0] = v.x; o[1] = v.y; }
+};
+template <> struct RawRow<4, true> {
+  uint2 v;
+  __device__ __forceinline__ void load(const void *b, long row, int D, int lane) {
+    v = __ldg(reinterpret_cast<const uint2 *>(reinterpret_cast<const __nv_bfloat16 *>(b) + row * D + lane * 4));
+  }
+  __device__ __forceinline__ void get(float (&o)[4]) const {
+    o[0] = __uint_as_float(v.x << 16); o[1] = __uint_as_float(v.x & 0xFFFF0000u);
+    o[2] = __uint_as_float(v.y << 16); o[3] = __uint_as_float(v.y & 0xFFFF0000u);
+  }
+};
+template <> struct RawRow<2, true> {
+  uint32_t v;
+  __device__ __forceinline__ void load(const void *b, long row, int D, int lane) {
+    v = __ldg(reinterpret_cast<const unsigned int *>(reinterpret_cast<const __nv_bfloat16 *>(b) + row * D + lane * 2));
+  }
+  __device__ __forceinline__ void get(float (&o)[2]) const {
+    o[0] = __uint_as_float(v << 16); o[1] = __uint_as_float(v & 0xFFFF0000u);
+  }
+};
+
 template <int V, bool BF>
 __device__ __forceinline__ void store_row_t(void *base, long row, int D, int lane, const float (&v)[V]) {
   if constexpr (BF) {
@@ -439,8 +476,8 @@ __device__ __forceinline__ void store_row_t(void *base, long row, int D, int lan
   }
 }
 
-template <int D, int G, bool RP, bool BF = false>
-__global__ void __launch_bounds__(NT, G == 4 ? 4 : 3) gather_segsum_v2_kernel(
+template <int D, int G, bool RP, bool BF = false, bool PF = false>
+__global__ void __launch_bounds__(NT, (BF ? G <= 8 : G == 4) ? 4 : 3) gather_segsum_v2_kernel(
     const void *__restrict__ g, const void *__restrict__ hbar,
     const int32_t *__restrict__ in_ptr, const int32_t *__restrict__ in_src, int N, int mean,
     float slope, void *__restrict__ h_out, const int32_t *__restrict__ node_graph,
@@ -450,6 +487,8 @@ __global__ void __launch_bounds__(NT, G == 4 ? 4 : 3) gather_segsum_v2_kernel(
   const int lane = threadIdx.x & 31;
   const long nw = (long(gridDim.x) * NT) / 32;
   long t0 = (blockIdx.x * long(NT) + threadIdx.x) / 32 * NPW;
+  pdl_trigger();
+  pdl_wait();
   if (t0 >= N) return;
   auto load_ptr = [&](long t) {
     const int n = int(min(long(NPW), N - t));
@@ -504,14 +543,27 @@ __global__ void __launch_bounds__(NT, G == 4 ? 4 : 3) gather_segsum_v2_kernel(
     for (int base = e_beg; base < e_end; base += 32) {
       const int cnt = min(32, e_end - base);
       if (base > e_beg) s_l = lane < cnt ? __ldg(in_src + base + lane) : 0;
-      for (int j = 0; j < cnt; j += G) {
-        float gv[G][V], hv[G][V];
+      RawRow<V, BF> gr[G], hr[G], gn[G], hn[G];
+      auto issue = [&](int j, RawRow<V, BF> (&ga)[G], RawRow<V, BF> (&ha)[G]) {
 #pragma unroll
         for (int u = 0; u < G; ++u) {
           const int kk = min(j + u, cnt - 1);
           const int sidx = __shfl_sync(0xffffffffu, s_l, kk);
-          load_row<V, BF>(g, long(base + kk), D, lane, gv[u]);
-          load_row<V, BF>(hbar, long(sidx), D, lane, hv[u]);
+          ga[u].load(g, long(base + kk), D, lane);
+          ha[u].load(hbar, long(sidx), D, lane);
+        }
+      };
+      if (PF) issue(0, gn, hn);
+      for (int j = 0; j < cnt; j += G) {
+        if (PF) {
+#pragma unroll
+          for (int u = 0; u < G; ++u) {
+            gr[u] = gn[u];
+            hr[u] = hn[u];
+          }
+          if (j + G < cnt) issue(j + G, gn, hn);        // next round in flight while this one sums
+        } else {
+          issue(j, gr, hr);
         }
         if (!next_src_issued && t1 < N) {                      // next chunk's first sources
           const int nb = __shfl_sync(0xffffffffu, ptr_n, 0);
@@ -529,8 +581,11 @@ __global__ void __launch_bounds__(NT, G == 4 ? 4 : 3) gather_segsum_v2_kernel(
               ++node;
               seg_end = __shfl_sync(0xffffffffu, ptr_l, node + 1);
             }
+            float gv[V], hv[V];
+            gr[u].get(gv);
+            hr[u].get(hv);
 #pragma unroll
-            for (int c = 0; c < V; ++c) acc[c] = fmaf(gv[u][c], hv[u][c], acc[c]);
+            for (int c = 0; c < V; ++c) acc[c] = fmaf(gv[c], hv[c], acc[c]);
           }
         }
       }
@@ -575,6 +630,8 @@ __global__ void __launch_bounds__(RO_WARPS * 32) readout_head_kernel(
     float *__restrict__ c_out, float *__restrict__ yhat, int chunk) {
   constexpr int V = D / 32;
   extern __shared__ float sm[];
+  pdl_trigger();
+  pdl_wait();
   float *part = sm;                    // [RO_WARPS][D]
   float *rs = part + RO_WARPS * D;     // [D]
   float *os = rs + D;                  // [d_h]
@@ -1206,11 +1263,17 @@ static int gather_impl(const occu_ctx *ctx, const DevCsr &csr, const float *g, c
   } else {
     const int grid = grid_for(long(csr.N) * 4, NT, occ * ctx->num_sms);
     if (variant == 1) {
-      if (rpart) gather_segsum_v2_kernel<D, 4, true><<<grid, NT, 0, st>>>(OCCU_GATHER_ARGS);
-      else gather_segsum_v2_kernel<D, 4, false><<<grid, NT, 0, st>>>(OCCU_GATHER_ARGS);
+      if (rpart) launch_pdl(ctx->pdl & 2, gather_segsum_v2_kernel<D, 4, true>, grid, NT, 0, st, OCCU_GATHER_ARGS);
+      else launch_pdl(ctx->pdl & 2, gather_segsum_v2_kernel<D, 4, false>, grid, NT, 0, st, OCCU_GATHER_ARGS);
+    } else if (variant == 3) {
+      if (rpart) launch_pdl(ctx->pdl & 2, gather_segsum_v2_kernel<D, 4, true, false, true>, grid, NT, 0, st, OCCU_GATHER_ARGS);
+      else launch_pdl(ctx->pdl & 2, gather_segsum_v2_kernel<D, 4, false, false, true>, grid, NT, 0, st, OCCU_GATHER_ARGS);
+    } else if (variant == 4) {
+      if (rpart) launch_pdl(ctx->pdl & 2, gather_segsum_v2_kernel<D, 2, true, false, true>, grid, NT, 0, st, OCCU_GATHER_ARGS);
+      else launch_pdl(ctx->pdl & 2, gather_segsum_v2_kernel<D, 2, false, false, true>, grid, NT, 0, st, OCCU_GATHER_ARGS);
     } else {
-      if (rpart) gather_segsum_v2_kernel<D, 8, true><<<grid, NT, 0, st>>>(OCCU_GATHER_ARGS);
-      else gather_segsum_v2_kernel<D, 8, false><<<grid, NT, 0, st>>>(OCCU_GATHER_ARGS);
+      if (rpart) launch_pdl(ctx->pdl & 2, gather_segsum_v2_kernel<D, 8, true>, grid, NT, 0, st, OCCU_GATHER_ARGS);
+      else launch_pdl(ctx->pdl & 2, gather_segsum_v2_kernel<D, 8, false>, grid, NT, 0, st, OCCU_GATHER_ARGS);
     }
   }
 #undef OCCU_GATHER_ARGS
@@ -1224,14 +1287,28 @@ static int gather_bf16_impl(const occu_ctx *ctx, const DevCsr &csr, const void *
                             void *h_out, float *rpart, cudaStream_t st) {
   if (csr.N <= 0) return 0;
   const int mean = ctx->cfg.aggr == OCCU_AGGR_MEAN;
-  const int grid = grid_for(long(csr.N) * 4, NT, 8 * ctx->num_sms);
+  static const int gsel = [] {
+    const char *e = getenv("OCCU_GATHER_G");
+    return e ? atoi(e) : 4;
+  }();
+  static const int bps = [] {
+    const char *e = getenv("OCCU_GATHER_BPS");
+    return e ? atoi(e) : 8;
+  }();
+  const int grid = grid_for(long(csr.N) * 4, NT, bps * ctx->num_sms);
   OCCU_PROF_BEGIN(ctx, "gather_segsum", st);
-  if (rpart)
-    gather_segsum_v2_kernel<D, 4, true, true><<<grid, NT, 0, st>>>(
-        g, hbar, csr.in_ptr, csr.in_src, csr.N, mean, ctx->cfg.slope, h_out, csr.node_graph, rpart);
-  else
-    gather_segsum_v2_kernel<D, 4, false, true><<<grid, NT, 0, st>>>(
-        g, hbar, csr.in_ptr, csr.in_src, csr.N, mean, ctx->cfg.slope, h_out, csr.node_graph, rpart);
+#define OCCU_GB_ARGS g, hbar, csr.in_ptr, csr.in_src, csr.N, mean, ctx->cfg.slope, h_out, csr.node_graph, rpart
+  if (gsel == 4) {
+    if (rpart) launch_pdl(ctx->pdl & 64, gather_segsum_v2_kernel<D, 4, true, true>, grid, NT, 0, st, OCCU_GB_ARGS);
+    else launch_pdl(ctx->pdl & 64, gather_segsum_v2_kernel<D, 4, false, true>, grid, NT, 0, st, OCCU_GB_ARGS);
+  } else if (gsel == 2) {
+    if (rpart) launch_pdl(ctx->pdl & 64, gather_segsum_v2_kernel<D, 2, true, true, true>, grid, NT, 0, st, OCCU_GB_ARGS);
+    else launch_pdl(ctx->pdl & 64, gather_segsum_v2_kernel<D, 2, false, true, true>, grid, NT, 0, st, OCCU_GB_ARGS);
+  } else {
+    if (rpart) launch_pdl(ctx->pdl & 64, gather_segsum_v2_kernel<D, 4, true, true, true>, grid, NT, 0, st, OCCU_GB_ARGS);
+    else launch_pdl(ctx->pdl & 64, gather_segsum_v2_kernel<D, 4, false, true, true>, grid, NT, 0, st, OCCU_GB_ARGS);
+  }
+#undef OCCU_GB_ARGS
   OCCU_PROF_END(ctx);
   LAUNCH_CHECK();
   return 1;
@@ -1283,8 +1360,8 @@ int launch_readout_head(const occu_ctx *ctx, const DevCsr &csr, const float *h, 
   OCCU_PROF_BEGIN(ctx, "readout_head", st);
 #define OCCU_RO_ARGS h, csr.node_off, cf.d_h, params + L.W_1, params + L.b_1, params + L.w_2, \
     params + L.b_2, cf.slope, r, c, yhat, chunked ? 8 : 0
-  if (cf.d == 64) readout_head_kernel<64><<<csr.B, RO_WARPS * 32, smem, st>>>(OCCU_RO_ARGS);
-  else readout_head_kernel<128><<<csr.B, RO_WARPS * 32, smem, st>>>(OCCU_RO_ARGS);
+  if (cf.d == 64) launch_pdl(ctx->pdl & 8, readout_head_kernel<64>, csr.B, RO_WARPS * 32, smem, st, OCCU_RO_ARGS);
+  else launch_pdl(ctx->pdl & 8, readout_head_kernel<128>, csr.B, RO_WARPS * 32, smem, st, OCCU_RO_ARGS);
 #undef OCCU_RO_ARGS
   OCCU_PROF_END(ctx);
   LAUNCH_CHECK();

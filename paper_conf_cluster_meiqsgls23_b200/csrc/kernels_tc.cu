@@ -251,14 +251,7 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
   Smem s = carve(smem_raw, D, K);
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
 
-  // ---- weights: prebuilt fp16x2 images (wimage_kernel), bulk-copied by the producer ----
-  const int fexp = __ldg(a.wfexp);
-  const bool noshift = __ldg(a.wfexp + 1) != 0;
-  if (EPI == EPI_NODE)
-    for (int i = threadIdx.x; i < D; i += NTH) {
-      s.avec[i] = a.a_s[i];
-      s.avec[D + i] = a.a_d[i];
-    }
+  pdl_trigger();
   if (threadIdx.x == 0) {
     for (int j = 0; j < 2; ++j) {
       tc::mbar_init(s.full + j, 1);
@@ -273,6 +266,15 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
     tc::fence_mbar_init();
   }
   if (warp == 1) tc::tmem_alloc<TMEM_COLS>(s.tmem_slot);
+  pdl_wait();                              // predecessor's writes visible from here on
+  // ---- weights: prebuilt fp16x2 images (wimage_kernel), bulk-copied by the producer ----
+  const int fexp = __ldg(a.wfexp);
+  const bool noshift = __ldg(a.wfexp + 1) != 0;
+  if (EPI == EPI_NODE)
+    for (int i = threadIdx.x; i < D; i += NTH) {
+      s.avec[i] = a.a_s[i];
+      s.avec[D + i] = a.a_d[i];
+    }
   // generic-proxy smem writes (weight images) must be visible to the async proxy (MMA)
   asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
   tc::fence_before_sync();
@@ -1202,6 +1204,8 @@ struct WImageJob {
 };
 
 __global__ void __launch_bounds__(256) wimage_kernel(const WImageJob *__restrict__ jobs) {
+  pdl_trigger();
+  pdl_wait();
   const WImageJob jb = jobs[blockIdx.x];
   const int D = jb.D, K = jb.K, Kpad = kpad_of(K);
   __shared__ float red[8];
@@ -1275,6 +1279,8 @@ __global__ void __launch_bounds__(256) edge_small_kernel(
     float *__restrict__ e_out, float *__restrict__ e0_out) {
   constexpr int V = D / 32;                 // channels per lane
   extern __shared__ float wsm[];            // [Ke][D] = W_eᵀ
+  pdl_trigger();
+  pdl_wait();
   for (int i = threadIdx.x; i < D * Ke; i += blockDim.x) wsm[(i % Ke) * D + i / Ke] = W_e[i];
   __syncthreads();
   const int lane = threadIdx.x & 31;
@@ -1629,7 +1635,7 @@ int tc_prepare_weights(occu_ctx *ctx, cudaStream_t st) {
                       cudaMemcpyHostToDevice, st) != cudaSuccess)
     return -int(cudaErrorInvalidValue);
   OCCU_PROF_BEGIN(ctx, "wimage", st);
-  wimage_kernel<<<int(jobs.size()), 256, 0, st>>>(ctx->wjobs.as<WImageJob>());
+  launch_pdl(ctx->pdl & 32, wimage_kernel, int(jobs.size()), 256, 0, st, ctx->wjobs.as<WImageJob>());
   OCCU_PROF_END(ctx);
   TC_CHECK();
   ctx->wimg_version = ctx->params_version;
@@ -1653,7 +1659,7 @@ static int launch_rowgemm(const occu_ctx *ctx, const RowGemmArgs &ra, const char
   CUtensorMap tmap;
   if (!encode_rows_map(&tmap, ra.A, ra.R, ra.K)) return -int(cudaErrorInvalidValue);
   OCCU_PROF_BEGIN(ctx, name, st);
-  rowgemm_kernel<D, EPI><<<grid, NTH, smem, st>>>(tmap, ra);
+  launch_pdl(ctx->pdl & 1, rowgemm_kernel<D, EPI>, grid, NTH, smem, st, tmap, ra);
   OCCU_PROF_END(ctx);
   TC_CHECK();
   return 1;
@@ -1729,11 +1735,11 @@ static int tc_forward_layer_impl(const occu_ctx *ctx, const DevCsr &csr, int lay
       const int grid = int(std::min<long>((long(csr.E) + 255) / 256, 8L * ctx->num_sms));
       OCCU_PROF_BEGIN(ctx, "edge_small", st);
       if (a.Ke <= 4)
-        edge_small_kernel<D, 4><<<grid, 256, D * a.Ke * 4, st>>>(
-            a.e_in, a.Ke, a.W_e, a.p, a.q, csr.in_src, csr.in_dst, a.e_eid, csr.E, a.e_out, a.e0_out);
+        launch_pdl(ctx->pdl & 4, edge_small_kernel<D, 4>, grid, 256, D * a.Ke * 4, st, a.e_in, a.Ke, a.W_e,
+                   a.p, a.q, csr.in_src, csr.in_dst, a.e_eid, csr.E, a.e_out, a.e0_out);
       else
-        edge_small_kernel<D, 16><<<grid, 256, D * a.Ke * 4, st>>>(
-            a.e_in, a.Ke, a.W_e, a.p, a.q, csr.in_src, csr.in_dst, a.e_eid, csr.E, a.e_out, a.e0_out);
+        launch_pdl(ctx->pdl & 4, edge_small_kernel<D, 16>, grid, 256, D * a.Ke * 4, st, a.e_in, a.Ke, a.W_e,
+                   a.p, a.q, csr.in_src, csr.in_dst, a.e_eid, csr.E, a.e_out, a.e0_out);
       OCCU_PROF_END(ctx);
       TC_CHECK();
       ++n;

@@ -6,6 +6,7 @@
 #include <stdint.h>
 
 #include <string>
+#include <utility>
 #include <vector>
 
 #include "../../include/occu.h"
@@ -90,6 +91,10 @@ struct occu_ctx {
   bool keep = false;
   int path = 0;            // 0: tensor cores, 1: CUDA-core SIMT FP32, 2: tensor cores + fused aggregation
   int l2_order = 1;        // alternate row-walk direction between producer/consumer kernels (L2 reuse)
+  // programmatic dependent launch, per kernel family (bit mask, OCCU_PDL): 1 FP32 row-GEMMs,
+  // 2 FP32 gather, 4 layer-1 edge, 8 readout, 16 BF16 row-GEMMs, 32 weight images, 64 BF16
+  // gather.  Default from A/B runs on CFG2: the FP32 gather and the readout lose with it.
+  int pdl = 1 | 4 | 16 | 32 | 64;
   int fuse_edge_gate = 0;  // path 0: edge transform + gate in one kernel (edgegate_kernel), OCCU_FUSE_EG=1
   occu::DevBuf wimg, wjobs, wfexp;   // prebuilt tensor-core weight images (per parameter version)
   int64_t params_version = 0, wimg_version = -1;
@@ -109,6 +114,33 @@ struct occu_ctx {
 };
 
 namespace occu {
+
+// ---- programmatic dependent launch (PDL) -------------------------------------
+// Kernels launched with launch_pdl may start (prologue: barriers, TMEM, tensor-map
+// prefetch) while their predecessor drains; every such kernel calls pdl_trigger()
+// first and pdl_wait() before its first global-memory access, so it observes all of
+// the predecessor's writes (and, transitively, everything earlier on the stream).
+#ifdef __CUDACC__
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+__device__ __forceinline__ void pdl_trigger() {
+  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+}
+template <class... KArgs, class... Args>
+cudaError_t launch_pdl(bool pdl, void (*kern)(KArgs...), dim3 grid, dim3 block, size_t smem,
+                       cudaStream_t st, Args &&...args) {
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = grid;
+  cfg.blockDim = block;
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = st;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[0].val.programmaticStreamSerializationAllowed = pdl ? 1 : 0;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  return cudaLaunchKernelEx(&cfg, kern, std::forward<Args>(args)...);
+}
+#endif
 
 #define OCCU_PROF_BEGIN(ctx, name, st) \
   do { if ((ctx)->prof.on) (ctx)->prof.begin(name, st); } while (0)

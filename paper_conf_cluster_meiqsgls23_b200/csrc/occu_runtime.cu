@@ -406,6 +406,7 @@ occu_status occu_create(occu_ctx **out, const occu_config *cfg, int cuda_device,
   cudaDeviceGetAttribute(&ctx->num_sms, cudaDevAttrMultiProcessorCount, cuda_device);
   if (const char *e = getenv("OCCU_L2_ORDER")) ctx->l2_order = atoi(e);   // A/B switches
   if (const char *e = getenv("OCCU_FUSE_EG")) ctx->fuse_edge_gate = atoi(e);
+  if (const char *e = getenv("OCCU_PDL")) ctx->pdl = atoi(e);
   const size_t pb = (ctx->layout.total + 1) * 4;
   if (ctx->params.ensure(pb) != cudaSuccess || ctx->grads.ensure(pb) != cudaSuccess ||
       ctx->adam_m.ensure(pb) != cudaSuccess || ctx->adam_v.ensure(pb) != cudaSuccess) {
