@@ -313,3 +313,44 @@ def test_training_trajectory_matches_oracle():
     # allow a few sign flips of near-zero gradients (<= 2 lr each)
     assert np.all(np.abs(w - wr)[slack] <= 2 * lr * 10 + 1e-6)
     assert slack.mean() < 0.01
+
+
+def test_cfg3_full_size_training_properties():
+    """BASELINE configs[2] at full size (512 BERT-base / GPT-2 training graphs, ~1.5 M nodes,
+    ~2.4 M edges, L=3, d=128), FP32 path as bench/train would run it.  The oracle cannot
+    run the full-batch backward in seconds, so: (i) ŷ of sampled graphs vs the oracle one by
+    one; (ii) the loss equals (1/B) Σ (ŷ_b - y_b)² of the library's own predictions; (iii) the
+    data-parallel identity at full size: the gradient of the batch equals the sum of the
+    gradients of its two halves (loss scaled by the global B, R15)."""
+    import torch
+    c = mk(3, 128)
+    b = configs.cfg3(512)
+    flat = weights.init_flat(wcfg(c), 42)
+    m = occu.Model(c)
+    m.set_params(flat)
+    dev = torch.device("cuda", 0)
+
+    def dev_batch(bb):
+        return (m.to_device(occu.pack(bb.graphs)), torch.from_numpy(bb.node_feat).to(dev),
+                torch.from_numpy(bb.edge_feat).to(dev), torch.from_numpy(bb.targets).to(dev))
+
+    csr, nf, ef, yt = dev_batch(b)
+    y = m.predict(csr, nf, ef)
+    torch.cuda.synchronize()
+    y = y.cpu().numpy().astype(np.float64)
+    params = oracle.unflatten(ocfg(c), flat.astype(np.float64))
+    for gi in (0, 255, 256, 511):
+        s = b.subset([gi])
+        yr = oracle.predict(params, ocfg(c), s.graphs, s.node_feat, s.edge_feat)
+        assert abs(y[gi] - yr[0]) <= TOL * max(abs(yr[0]), 1e-2), gi
+    loss = m.compute_grads(csr, nf, ef, yt)
+    g_full = m.get_grads()
+    want = float(np.mean((y - b.targets.astype(np.float64)) ** 2))
+    assert abs(loss - want) <= 1e-5 * want
+    g_sum = np.zeros_like(g_full, dtype=np.float64)
+    for half in (list(range(0, 256)), list(range(256, 512))):
+        hb = b.subset(half)
+        hc, hn, he, hy = dev_batch(hb)
+        m.compute_grads(hc, hn, he, hy, global_num_graphs=512)
+        g_sum += m.get_grads().astype(np.float64)
+    assert rel(g_full, g_sum) <= 1e-5, rel(g_full, g_sum)
