@@ -602,6 +602,64 @@ __global__ void __launch_bounds__(NT, (BF ? G <= 8 : G == 4) ? 4 : 3) gather_seg
   }
 }
 
+// ---------------------------------------------------------------------------
+// a10, gate / message backward with the forward's gates g (no recompute): per edge k,
+//   dm = dA[t_k] (LReLU' and ÷deg already applied), MG = dm ⊙ g, dg = dm ⊙ h̄[s_k],
+//   DV = g ⊙ (dg − ⟨g, dg⟩)          (softmax backward; ⟨·,·⟩ accumulated in float64)
+// A warp takes 32 consecutive in-CSR edges, four at a time with all row loads of the
+// four in flight; lane = D/32 channels; the dot is a fixed-order butterfly.
+// ---------------------------------------------------------------------------
+template <int D>
+__global__ void __launch_bounds__(NT) gate_bwd_stream_kernel(
+    const float *__restrict__ g, const float *__restrict__ dA, const float *__restrict__ hbar,
+    const int32_t *__restrict__ in_src, const int32_t *__restrict__ in_dst, int E,
+    float *__restrict__ MG, float *__restrict__ DV) {
+  constexpr int V = D / 32;
+  constexpr int G = 4;
+  const int lane = threadIdx.x & 31;
+  const long nwarps = long(gridDim.x) * (NT / 32);
+  for (long k0 = (blockIdx.x * long(NT / 32) + threadIdx.x / 32) * 32; k0 < E; k0 += nwarps * 32) {
+    const int cnt = int(min(32L, E - k0));
+    const int s_l = lane < cnt ? __ldg(in_src + k0 + lane) : 0;
+    const int t_l = lane < cnt ? __ldg(in_dst + k0 + lane) : 0;
+    for (int j = 0; j < cnt; j += G) {
+      RawRow<V, false> gr[G], dr[G], hr[G];
+#pragma unroll
+      for (int u = 0; u < G; ++u) {
+        const int kk = min(j + u, cnt - 1);
+        gr[u].load(g, k0 + kk, D, lane);
+        dr[u].load(dA, __shfl_sync(0xffffffffu, t_l, kk), D, lane);
+        hr[u].load(hbar, __shfl_sync(0xffffffffu, s_l, kk), D, lane);
+      }
+#pragma unroll
+      for (int u = 0; u < G; ++u) {
+        if (j + u >= cnt) break;                       // warp-uniform
+        float gv[V], dv[V], hv[V], dg[V];
+        gr[u].get(gv);
+        dr[u].get(dv);
+        hr[u].get(hv);
+        double dot = 0.0;
+#pragma unroll
+        for (int c = 0; c < V; ++c) {
+          dg[c] = dv[c] * hv[c];
+          dot = fma(double(gv[c]), double(dg[c]), dot);
+        }
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) dot += __shfl_xor_sync(0xffffffffu, dot, o);
+        const float dotf = float(dot);
+        float mg[V], dvv[V];
+#pragma unroll
+        for (int c = 0; c < V; ++c) {
+          mg[c] = dv[c] * gv[c];
+          dvv[c] = gv[c] * (dg[c] - dotf);
+        }
+        store_row<V>(MG + (k0 + j + u) * D + lane * V, mg);
+        store_row<V>(DV + (k0 + j + u) * D + lane * V, dvv);
+      }
+    }
+  }
+}
+
 // e0[k] = edge_feat[in_eid[k]]  (a1)
 __global__ void permute_rows_kernel(const float *__restrict__ src, const int32_t *__restrict__ idx,
                                     int rows, int width, float *__restrict__ dst) {
@@ -1468,10 +1526,20 @@ static int backward_layer_impl(occu_ctx *ctx, const DevCsr &csr, const BwdLayerA
   const bool tc = ctx->path != 1 && tc_supported(cf);
   int r;
   if (tc && csr.E > 0) {
-    // a10 on tensor cores: g recompute + softmax backward, W_mᵀ dv, z recompute + σ', W_eᵀ dz
-    if ((r = launch_bwd_gate_tc(ctx, csr, i, a.e, a.dh, nullptr, a.hbar, w.MG.as<float>(),
-                                w.DV.as<float>(), st)) < 0) return r;
-    n += r;
+    // a10: softmax / message backward (streaming with the saved gates, else g recomputed on
+    // tensor cores), W_mᵀ dv, z recompute + σ', W_eᵀ dz on tensor cores
+    if (a.g) {
+      OCCU_PROF_BEGIN(ctx, "gate_bwd", st);
+      gate_bwd_stream_kernel<D><<<grid_for((long(csr.E) + 31) / 32, NT / 32, 8 * sms), NT, 0, st>>>(
+          a.g, a.dh, a.hbar, csr.in_src, csr.in_dst, csr.E, w.MG.as<float>(), w.DV.as<float>());
+      OCCU_PROF_END(ctx);
+      LAUNCH_CHECK();
+      ++n;
+    } else {
+      if ((r = launch_bwd_gate_tc(ctx, csr, i, a.e, a.dh, nullptr, a.hbar, w.MG.as<float>(),
+                                  w.DV.as<float>(), st)) < 0) return r;
+      n += r;
+    }
     if ((r = launch_plain_tc(ctx, w.DV.as<float>(), D, csr.E, 3, i, a.de_out, de,
                              "de_tc", st)) < 0) return r;
     n += r;

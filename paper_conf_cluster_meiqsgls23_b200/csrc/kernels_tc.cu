@@ -1348,7 +1348,7 @@ __global__ void __launch_bounds__(256) edge_small_kernel(
 // owns a contiguous row range; partials are reduced in fixed split order afterwards.
 // ---------------------------------------------------------------------------
 constexpr int WG_NS = 3;                  // pipeline stages of 32 rows
-constexpr int WG_NTH = 192;               // warp0 TMA, warp1 MMA, warps 2-5 lo / epilogue
+constexpr int WG_NTH = 320;               // warp0 TMA, warp1 MMA, warps 2-9 lo / epilogue
 
 __global__ void __launch_bounds__(WG_NTH, 1)
 wgrad_tc_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant__ CUtensorMap ymap,
@@ -1370,7 +1370,7 @@ wgrad_tc_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant_
   if (threadIdx.x == 0) {
     for (int j = 0; j < WG_NS; ++j) {
       tc::mbar_init(full + j, 1);
-      tc::mbar_init(lo_ready + j, 128);
+      tc::mbar_init(lo_ready + j, 256);
       tc::mbar_init(empty + j, 1);
     }
     tc::mbar_init(done, 1);
@@ -1424,30 +1424,37 @@ wgrad_tc_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant_
       __syncwarp();
     }
   } else {
-    const int t = threadIdx.x - 64;              // 0..127
+    const int t = threadIdx.x - 64;              // 0..255
     for (int i = 0; i < nst; ++i) {
       const int j = i % WG_NS;
       tc::mbar_wait(full + j, (i / WG_NS) & 1);
       uint8_t *st = stage(j);
       const long r0 = rb + long(i) * 32;
-      // X raw -> X lo (boxes 0..nbx), Y raw -> Y lo; rows beyond this CTA's range -> 0
-      for (int f = t; f < 2 * 4 * 256; f += 128) {          // 2 operands x 4 boxes x 256 float4
-        const int op = f >> 10, b = (f >> 8) & 3, q4 = f & 255;
+      // X raw -> X lo (boxes 0..nbx), Y raw -> Y lo; rows beyond this CTA's range -> 0.
+      // 2 operands x 4 boxes x 256 float4 = 8 per thread, all loads issued before use.
+      float4 v[8];
+#pragma unroll
+      for (int it = 0; it < 8; ++it) {
+        const int f = t + it * 256, op = f >> 10, b = (f >> 8) & 3, q4 = f & 255;
+        v[it] = make_float4(0.f, 0.f, 0.f, 0.f);
+        if (b < (op == 0 ? nbx : nby))
+          v[it] = reinterpret_cast<const float4 *>(st + op * 32768 + b * 4096)[q4];
+      }
+#pragma unroll
+      for (int it = 0; it < 8; ++it) {
+        const int f = t + it * 256, op = f >> 10, b = (f >> 8) & 3, q4 = f & 255;
         if (b >= (op == 0 ? nbx : nby)) continue;
-        float4 *raw = reinterpret_cast<float4 *>(st + op * 32768 + b * 4096) + q4;
-        float4 *lo = reinterpret_cast<float4 *>(st + op * 32768 + 16384 + b * 4096) + q4;
-        const int rr = q4 >> 3;                               // 8 float4 per 128-byte row
-        float4 v = *raw;
-        if (r0 + rr >= re) {
-          v = make_float4(0.f, 0.f, 0.f, 0.f);
-          *raw = v;
+        float4 x = v[it];
+        if (r0 + (q4 >> 3) >= re) {                       // 8 float4 per 128-byte row
+          x = make_float4(0.f, 0.f, 0.f, 0.f);
+          reinterpret_cast<float4 *>(st + op * 32768 + b * 4096)[q4] = x;
         }
         float4 l;
-        l.x = v.x - __uint_as_float(__float_as_uint(v.x) & 0xFFFFE000u);
-        l.y = v.y - __uint_as_float(__float_as_uint(v.y) & 0xFFFFE000u);
-        l.z = v.z - __uint_as_float(__float_as_uint(v.z) & 0xFFFFE000u);
-        l.w = v.w - __uint_as_float(__float_as_uint(v.w) & 0xFFFFE000u);
-        *lo = l;
+        l.x = x.x - __uint_as_float(__float_as_uint(x.x) & 0xFFFFE000u);
+        l.y = x.y - __uint_as_float(__float_as_uint(x.y) & 0xFFFFE000u);
+        l.z = x.z - __uint_as_float(__float_as_uint(x.z) & 0xFFFFE000u);
+        l.w = x.w - __uint_as_float(__float_as_uint(x.w) & 0xFFFFE000u);
+        reinterpret_cast<float4 *>(st + op * 32768 + 16384 + b * 4096)[q4] = l;
       }
       asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
       tc::mbar_arrive(lo_ready + j);
@@ -1457,10 +1464,11 @@ wgrad_tc_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant_
       tc::mbar_wait(done, 0);
       tc::fence_after_sync();
     }
-    const int q = warp & 3, row = q * 32 + lane;
+    const int q = warp & 3, row = q * 32 + lane, hh = (warp - 2) >> 2;
     const uint32_t lane_base = tmem + (uint32_t(q * 32) << 16);
     float *out = partial + long(blockIdx.x) * A * Bn + long(row) * Bn;
-    for (int c0 = 0; c0 < Npad; c0 += 16) {
+    const int chalf = (Npad / 16 + 1) / 2 * 16;             // two warps per TMEM lane quarter
+    for (int c0 = hh * chalf; c0 < min(Npad, (hh + 1) * chalf); c0 += 16) {
       uint32_t r[16];
       if (nst > 0) {
         tc::tmem_ld16(lane_base + c0, r);

@@ -43,6 +43,7 @@ struct Workspace {
   DevBuf csr;              // concatenated int32 CSR arrays for host-CSR calls
   DevBuf e0;               // edge features permuted to in-CSR order [E][F_e]
   std::vector<DevBuf> hbar, p, q, e, h;   // per layer
+  std::vector<DevBuf> gs;                 // per layer channel-softmax gates, kept for the backward (training)
   DevBuf g;                // [E][d] channel-softmax gates (scratch)
   DevBuf rpart;            // [N][d] readout chunk partials (rows written sparsely) when h_L is kept
   DevBuf r, c, yhat;       // [B][d], [B][d_h], [B]
@@ -201,6 +202,7 @@ struct BwdLayerArgs {
   const float *h_in; int K;           // h^{i-1} [N][K]
   const float *e_in; int Ke;          // e^{i-1} [E][Ke]
   const float *hbar, *p, *q, *e, *h;  // layer i saved
+  const float *g;                     // layer i gates saved by the forward (nullable: recompute)
   const float *dh;                    // [N][d] gradient w.r.t. h^i
   const float *de_out;                // [E][d] gradient w.r.t. e^i from layer i+1 (nullable)
   float *de_prev;                     // [E][Ke] (nullable at layer 0)

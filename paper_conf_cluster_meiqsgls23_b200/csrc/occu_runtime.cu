@@ -260,6 +260,11 @@ occu_status forward(occu_ctx *ctx, const DevCsr &csr, const float *nf, const flo
     a.hbar = w.hbar[i].as<float>(); a.p = w.p[i].as<float>(); a.q = w.q[i].as<float>();
     a.e_out = (!last || save_all) ? w.e[i].as<float>() : nullptr;
     a.g = w.g.as<float>();
+    if (save_all && tc && !bf && ctx->path == 0) {    // the backward reads the gates (no recompute)
+      if (w.gs.size() < size_t(c.L)) w.gs.resize(c.L);
+      CK(w.gs[i].ensure(size_t(csr.E) * c.d * 4), "alloc saved gates");
+      a.g = w.gs[i].as<float>();
+    }
     a.h_out = w.h[i].as<float>();
     if (tc) {
       a.e_out = w.e[i].as<float>();            // the gate kernel re-reads e'
@@ -368,6 +373,7 @@ occu_status grads_impl(occu_ctx *ctx, const occu_batch *batch, const float *targ
     a.Ke = L.de_in[i];
     a.hbar = w.hbar[i].as<float>(); a.p = w.p[i].as<float>(); a.q = w.q[i].as<float>();
     a.e = w.e[i].as<float>(); a.h = w.h[i].as<float>();
+    a.g = (ctx->path == 0 && w.gs.size() > size_t(i)) ? w.gs[i].as<float>() : nullptr;
     a.dh = w.dh.as<float>();
     a.de_out = i < c.L - 1 ? w.deB.as<float>() : nullptr;
     a.de_prev = i > 0 ? w.deB.as<float>() : nullptr;     // read-before-write ordering, see DESIGN
