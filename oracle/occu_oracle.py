@@ -231,13 +231,15 @@ def bf16_round(x):
     return b.view(np.float32).astype(np.float64)
 
 
-def forward_bf16(params, cfg, pk, node_feat, edge_feat):
+def forward_bf16(params, cfg, pk, node_feat, edge_feat, rnd=None):
     """Forward of OCCU_BF16: tensor-core GEMM operands (activations and W_u, W_e, W_m) are
     rounded to BF16 (R24); stored h̄, e', g, h are BF16 (R24); p, q come from the unrounded
     h̄ and, like α, σ, the softmax, the message product, the segment sums, the readout (over
     the unrounded last-layer h, R27) and the head, stay unrounded.  The layer-1 edge
-    transform with F_e <= 16 is a CUDA-core FP32 step, not a tensor-core GEMM (R27)."""
-    r16 = bf16_round
+    transform with F_e <= 16 is a CUDA-core FP32 step, not a tensor-core GEMM (R27).
+    ``rnd`` replaces the rounding function (tests pass the identity to recover forward()).
+    The saved fields are the ones the training backward of the mode reads (R28)."""
+    r16 = bf16_round if rnd is None else rnd
     slope = cfg["slope"]
     s_k, t_k = pk["in_src"].astype(np.int64), pk["in_dst"].astype(np.int64)
     N = pk["num_nodes"]
@@ -262,13 +264,17 @@ def forward_bf16(params, cfg, pk, node_feat, edge_feat):
         if cfg["aggr"] == AGGR_MEAN:
             A = A / np.maximum(deg, 1)[:, None]
         h_f = leaky_relu(A, slope)
-        layers.append(dict(hbar=hbar, p=p, q=q, e=e_new, g=g, h=r16(h_f), h_f32=h_f))
+        layers.append(dict(P=P, hbar=hbar, p=p, q=q, alpha=alpha, z=z, e=e_new, g=g, A=A,
+                           h=r16(h_f), h_f32=h_f))
         h, e = r16(h_f), e_new
     n_b = np.diff(pk["node_off"].astype(np.int64))
     r = segment_sum(layers[-1]["h_f32"], pk["node_graph"].astype(np.int64), pk["num_graphs"]) / n_b[:, None]
     c = r @ params["W_1"].T + params["b_1"]                       # P125 (R12)
-    yhat = leaky_relu(c, slope) @ params["w_2"] + params["b_2"][0]
-    return dict(layers=layers, r=r, c=c, yhat=yhat)
+    o = leaky_relu(c, slope)
+    yhat = o @ params["w_2"] + params["b_2"][0]
+    return dict(layers=layers, h0=np.asarray(node_feat, np.float64),
+                e0=np.asarray(edge_feat, np.float64)[pk["in_eid"].astype(np.int64)],
+                r=r, c=c, o=o, yhat=yhat)
 
 
 def predict(params, cfg, graphs, node_feat, edge_feat):
@@ -286,7 +292,9 @@ def mse_loss(yhat, y, global_batch=None):
 # --------------------------------------------------------------------------
 # Step BW: hand-derived backward of the forward above (reading A), float64.
 # --------------------------------------------------------------------------
-def backward(params, cfg, pk, fwd, y, global_batch=None):
+def backward(params, cfg, pk, fwd, y, global_batch=None, dsig=None):
+    """dsig(layer dict) -> σ'(y) per edge and channel; default e'(1 - e') (exact
+    derivative of σ at y = α z).  backward_bf16 passes e'·σ(-α z) (R28)."""
     slope = cfg["slope"]
     B = pk["num_graphs"]
     nb = B if global_batch is None else global_batch
@@ -328,7 +336,7 @@ def backward(params, cfg, pk, fwd, y, global_batch=None):
         de = dv @ W_m                      # de_k = W_m^T dv_k
         if de_out is not None:
             de = de + de_out
-        dyk = de * e * (1.0 - e)
+        dyk = de * (e * (1.0 - e) if dsig is None else dsig(lay))
         dalpha = np.sum(dyk * z, axis=1)
         dz = alpha[:, None] * dyk
         grads[f"W_e{i}"] = dz.T @ e_prev
@@ -349,6 +357,22 @@ def loss_and_grads(params, cfg, graphs, node_feat, edge_feat, y, global_batch=No
     pk = pack(graphs)
     fwd = forward(params, cfg, pk, node_feat, edge_feat)
     return backward(params, cfg, pk, fwd, y, global_batch)
+
+
+def backward_bf16(params, cfg, pk, fwd, y, global_batch=None):
+    """Step BW of OCCU_BF16 training (SURVEY §8(c) "Precision modes": all gradients FP32;
+    DESIGN.md R28): the hand-derived backward above evaluated on what the BF16 forward
+    saved — h̄, e', g and h as BF16 values, z as the mode computes it (BF16 operands on the
+    tensor cores), p, q, α, A and the head state unrounded — with the gradient GEMMs against
+    the unrounded weights and σ'(y) = e'·σ(-α z) (stored e', recomputed z)."""
+    return backward(params, cfg, pk, fwd, y, global_batch,
+                    dsig=lambda lay: lay["e"] * sigmoid(-lay["alpha"][:, None] * lay["z"]))
+
+
+def loss_and_grads_bf16(params, cfg, graphs, node_feat, edge_feat, y, global_batch=None):
+    pk = pack(graphs)
+    fwd = forward_bf16(params, cfg, pk, node_feat, edge_feat)
+    return backward_bf16(params, cfg, pk, fwd, y, global_batch)
 
 
 # --------------------------------------------------------------------------

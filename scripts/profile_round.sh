@@ -14,3 +14,7 @@ timeout 900 ncu --set full --clock-control none --import-source on \
   -k regex:"rowgemm_kernel<128, [45]>|wgrad_tc|split_reduce|node_bwd" -s 12 -c 8 -o gpurun_out/prof_train \
   python scripts/prof_driver.py --steps 3 --train > gpurun_out/prof_train.log 2>&1
 echo "train rc=$?" >> gpurun_out/prof_train.log
+timeout 900 ncu --set full --clock-control none --import-source on \
+  -k regex:"rowgemm|gather_segsum|edge_small" -s 7 -c 7 -o gpurun_out/prof_bf16 \
+  python scripts/prof_driver.py --steps 2 --bf16 > gpurun_out/prof_bf16.log 2>&1
+echo "bf16 rc=$?" >> gpurun_out/prof_bf16.log

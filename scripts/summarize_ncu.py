@@ -6,7 +6,7 @@ out = os.path.join(ROOT, "profiles")
 os.makedirs(out, exist_ok=True)
 
 def kname(full):
-    m = re.search(r"rowgemm_kernel<(\d+), (\d+)>", full)
+    m = re.search(r"rowgemm(?:_bf16)?_kernel<(\d+), (\d+)", full)
     if m:
         return ["node_tc", "edge_tc", "gate_tc", "plain_tc", "gatebwd_tc", "edgebwd_tc",
                 "gateagg_tc"][int(m.group(2))]
@@ -52,10 +52,9 @@ if os.path.exists(lp):
         print(f"  {k:16s} {a[0]:4d} {100*a[1]/tot:6.1f}% {a[2]/a[0]/1e6:9.1f} MB")
 
 # 2) full capture -> traffic per launch for the hot kernels
-traffic = {}
-lines = []
-for rep, drv in (("prof_full", "scripts/prof_driver.py (CFG2 inference)"),
-                 ("prof_train", "scripts/prof_driver.py --train (CFG2 training)")):
+def capture(reps):
+ traffic = {}
+ for rep, drv in reps:
   fp = os.path.join(ROOT, "gpurun_out", rep + ".ncu-rep")
   if os.path.exists(fp):
       raw = subprocess.run(["ncu", "-i", fp, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
@@ -89,9 +88,20 @@ for rep, drv in (("prof_full", "scripts/prof_driver.py (CFG2 inference)"),
                         "issue_active_pct": sum(x["issue_pct"] or 0 for x in lst) / n,
                         "registers": lst[0]["regs"],
                         "source": f"profiles/{tag}: ncu --set full, {drv}"}
+  # (end of one capture)
+ return traffic
+
+traffic = capture((("prof_full", "scripts/prof_driver.py (CFG2 inference)"),
+                   ("prof_train", "scripts/prof_driver.py --train (CFG2 training)")))
+traffic_bf = capture((("prof_bf16", "scripts/prof_driver.py --bf16 (CFG2 inference, OCCU_BF16)"),))
 json.dump(traffic, open(os.path.join(out, "traffic.json"), "w"), indent=1)
+if traffic_bf:
+    json.dump(traffic_bf, open(os.path.join(out, "traffic_bf16.json"), "w"), indent=1)
 with open(os.path.join(out, f"{tag}_ncu_summary.md"), "w") as f:
-    f.write(f"# {tag}: ncu --set full --clock-control none (serialised, cold-cache replays)\n\n")
+  for title, traffic in (("OCCU_FP32 (inference + training)", traffic), ("OCCU_BF16 inference", traffic_bf)):
+    if not traffic:
+        continue
+    f.write(f"# {tag}: ncu --set full --clock-control none (serialised, cold-cache replays), {title}\n\n")
     f.write("| kernel | launches | us/launch (ncu) | DRAM MB/launch | DRAM % peak | tensor pipe % | issue active % | regs |\n")
     f.write("|---|---|---|---|---|---|---|---|\n")
     for k, t in traffic.items():

@@ -460,3 +460,67 @@ def test_forward_bf16_rounds_where_the_mode_says():
         for k in ("hbar", "p", "e", "h"):
             ref = g["layers"][i][k]
             assert np.linalg.norm(lay[k] - ref) <= 2e-2 * np.linalg.norm(ref), (i, k)
+
+
+# ------------------------------------------ OCCU_BF16 training backward (R28)
+def test_backward_bf16_identity_rounding_is_the_plain_backward():
+    """With the rounding replaced by the identity, the BF16-mode forward is forward() and
+    backward_bf16's σ'(y) = e'·σ(-αz) equals e'(1 - e'): the gradients must be those of the
+    plain backward (itself pinned by finite differences and torch autograd above)."""
+    cfg = cfg_dict(L=3, F_n=80, F_e=4, d=16, d_h=8, aggr=0)
+    b = configs.random_dag_batch(5, 71, max_nodes=14, hub=True)
+    p = rand_params(cfg, 21)
+    for i in range(3):
+        p[f"W_u{i}"] *= 16
+    pk = oracle.pack(b.graphs)
+    ident = lambda x: np.asarray(x, np.float64)
+    fb = oracle.forward_bf16(p, cfg, pk, b.node_feat, b.edge_feat, rnd=ident)
+    fa = oracle.forward(p, cfg, pk, b.node_feat, b.edge_feat)
+    assert np.allclose(fb["yhat"], fa["yhat"], rtol=1e-13, atol=0)
+    lb, gb = oracle.backward_bf16(p, cfg, pk, fb, b.targets)
+    la, ga = oracle.backward(p, cfg, pk, fa, b.targets)
+    assert abs(lb - la) <= 1e-13 * la
+    for k in p:
+        assert np.linalg.norm(gb[k] - ga[k]) <= 1e-10 * np.linalg.norm(ga[k]) + 1e-300, k
+
+
+def test_backward_bf16_exact_when_rounding_is_exact():
+    """Integer X, W_u = I, a = 0, an integer W_m with equal row sums and BF16-representable
+    W_e / edge features make every BF16 rounding of the mode an identity (e' = 1/2, equal
+    logits so g = 1/d, dyadic h, z exact) while W_mᵀ dv, σ' and z still carry gradient
+    into a_s, a_d, so the BF16-mode gradients equal the float64 ones."""
+    d = 4
+    cfg = cfg_dict(L=2, F_n=d, F_e=d, d=d, d_h=d)
+    graphs = [(5, np.array([0, 0, 1, 2, 3], np.int32), np.array([1, 2, 3, 3, 4], np.int32))]
+    X = np.array([[1, 2, 3, 0], [0, 1, 0, 0], [2, 0, 0, 1], [0, 0, 0, 0], [1, 1, 1, 1]], np.float64)
+    rng = np.random.default_rng(3)
+    EF = oracle.bf16_round(rng.uniform(size=(5, d)))
+    Wm = np.array([[1, 2, 0, -1], [2, -1, 1, 0], [0, 1, -1, 2], [-1, 0, 2, 1]], np.float64)
+    p = toy_params(cfg, W_u0=np.eye(d), W_u1=np.eye(d), W_m0=Wm, W_m1=Wm.T.copy(),
+                   W_e0=oracle.bf16_round(rng.normal(size=(d, d))),
+                   W_e1=oracle.bf16_round(rng.normal(size=(d, d))),
+                   W_1=rng.normal(size=(d, d)), b_1=rng.normal(size=d), w_2=rng.normal(size=d))
+    y = np.array([0.3])
+    pk = oracle.pack(graphs)
+    lb, gb = oracle.backward_bf16(p, cfg, pk, oracle.forward_bf16(p, cfg, pk, X, EF), y)
+    la, ga = oracle.backward(p, cfg, pk, oracle.forward(p, cfg, pk, X, EF), y)
+    assert abs(lb - la) <= 1e-14 * la
+    for k in p:
+        assert np.allclose(gb[k], ga[k], rtol=1e-12, atol=1e-15), k
+    for k in ("W_m0", "W_m1", "a_s1", "a_d0", "W_u0"):      # dW_e = α·(...) = 0 here
+        assert np.linalg.norm(ga[k]) > 0, k
+
+
+def test_backward_bf16_within_the_bf16_budget():
+    """Real BF16 roundings: the mode's gradients approximate the exact ones to the BF16
+    budget (8 significant bits on stored activations, errors averaging over many terms)."""
+    cfg = cfg_dict(L=2, F_n=80, F_e=4, d=16, d_h=16)
+    b = configs.random_dag_batch(6, 45, max_nodes=20)
+    flat = weights.init_flat(weights.ModelConfig(L=2, d=16, d_h=16), 9)
+    p = oracle.unflatten(cfg, flat.astype(np.float64))
+    pk = oracle.pack(b.graphs)
+    lb, gb = oracle.backward_bf16(p, cfg, pk, oracle.forward_bf16(p, cfg, pk, b.node_feat, b.edge_feat), b.targets)
+    la, ga = oracle.backward(p, cfg, pk, oracle.forward(p, cfg, pk, b.node_feat, b.edge_feat), b.targets)
+    assert abs(lb - la) <= 2e-2 * la
+    for k in p:
+        assert np.linalg.norm(gb[k] - ga[k]) <= 3e-2 * np.linalg.norm(ga[k]), k
