@@ -183,6 +183,15 @@ occu_status occu_set_keep_intermediates(occu_ctx *ctx, int keep);
 /* Copy an intermediate of the last forward into host memory (float32; BF16
  * precision stores are widened).  bytes must equal the tensor size. */
 occu_status occu_get_tensor(occu_ctx *ctx, int32_t which, int32_t layer, void *host_dst, size_t bytes);
+/* Test hook for the weight-gradient GEMM of the backward (SURVEY §8(c) step BW: dW_m = DVᵀE',
+ * dW_e = DZᵀE_in, dW_u = dPᵀH_in): out[a][b] = Σ_{r<R} X[r][a]·Y[r][b] with the library's own
+ * kernels (deterministic split-K, fixed-order reduction), exactly as occu_train_step calls them.
+ * X: device FP32 [R][A]; Y: device [R][Bn], FP32, or BF16 when y_bf16 != 0 (OCCU_BF16
+ * training's stored activations; then A, Bn in {32..128}, multiples of 32 / 16); out: device
+ * FP32 [A][Bn].  Stream-ordered on the ctx stream.  EINVAL on NULL pointers or unsupported
+ * shapes; the ctx needs no weights. */
+occu_status occu_test_wgrad(occu_ctx *ctx, const float *X, int32_t A, const void *Y, int32_t Bn,
+                            int64_t R, int32_t y_bf16, float *out);
 /* Number of kernel launches issued by the last predict/train call. */
 int64_t occu_last_launch_count(const occu_ctx *ctx);
 

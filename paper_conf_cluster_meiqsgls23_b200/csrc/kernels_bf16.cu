@@ -9,6 +9,9 @@
 //   EPI_NODE : h̄ = LReLU(acc) -> BF16, p = h̄·a_s, q = h̄·a_d (FP32)        (a2, P141-P147)
 //   EPI_EDGE : e' = σ(α·acc), α = p[s] + q[t] -> BF16                       (a3, P145)
 //   EPI_GATE : g = softmax_c(acc) -> BF16                                   (a4, P149)
+//   EPI_EDGEBWD (training, R28): z = acc recomputed exactly as the forward's EPI_EDGE;
+//              dy = de ⊙ e' ⊙ σ(-αz) (BF16 e', FP32 de), dα = <dy, z> (float64), DZ = α dy
+//              -> FP32                                                      (a10, SURVEY §8(c) BW)
 // Input BF16 (layers >= 2): TMA writes the tile in the canonical SW128 K-major layout and
 // the MMA reads it straight from shared memory (no conversion pass).  Input FP32 (the
 // layer-1 node features): converter warps round it to BF16 into TMEM (".ts" form).
@@ -33,7 +36,7 @@ namespace {
 constexpr int TM = 128;
 constexpr int NTH = 832;
 constexpr int EPI0 = 10;
-constexpr int EPI_NODE = 0, EPI_EDGE = 1, EPI_GATE = 2;
+constexpr int EPI_NODE = 0, EPI_EDGE = 1, EPI_GATE = 2, EPI_EDGEBWD = 5;
 constexpr float LOG2E = 1.4426950408889634f;
 
 __device__ __forceinline__ float lrelu(float x, float s) { return x > 0.f ? x : s * x; }
@@ -60,7 +63,11 @@ struct BfArgs {
   const float *a_s, *a_d;    // NODE
   float *p, *q;              // NODE outputs
   const float *pin, *qin;    // EDGE
-  const int32_t *src, *dst;  // EDGE
+  const int32_t *src, *dst;  // EDGE, EDGEBWD
+  const __nv_bfloat16 *eb;   // EDGEBWD: e' [R][D]
+  const float *de;           // EDGEBWD: de [R][D]
+  float *outf;               // EDGEBWD: DZ [R][D]
+  float *dal;                // EDGEBWD: dα [R]
   float slope;
   int rev;
 };
@@ -98,6 +105,32 @@ __device__ __forceinline__ void warp_store_bf16(uint32_t *buf, __nv_bfloat16 *__
           *reinterpret_cast<const uint4 *>(buf + r * 12 + h * 4);
   }
   __syncwarp();
+}
+
+// Coalesced FP32 store of a 16-column chunk of the warp's 32 rows (thread = row), two
+// 16-row passes through a 16 x 20 per-warp buffer (full 64-byte row segments).
+__device__ __forceinline__ void warp_store_f32(float *buf, float *__restrict__ out, long wrow0,
+                                               int wrows, int c0, int D, const float (&v)[16],
+                                               int lane) {
+#pragma unroll
+  for (int h = 0; h < 2; ++h) {
+    if ((lane >> 4) == h) {
+      float *b = buf + (lane & 15) * 20;
+#pragma unroll
+      for (int u = 0; u < 16; u += 4)
+        *reinterpret_cast<float4 *>(b + u) = make_float4(v[u], v[u + 1], v[u + 2], v[u + 3]);
+    }
+    __syncwarp();
+#pragma unroll
+    for (int it = 0; it < 2; ++it) {
+      const int idx = it * 32 + lane, r = idx >> 2, c4 = (idx & 3) * 4;
+      const int rr = h * 16 + r;
+      if (rr < wrows)
+        *reinterpret_cast<float4 *>(out + (wrow0 + rr) * D + c0 + c4) =
+            *reinterpret_cast<const float4 *>(buf + r * 20 + c4);
+    }
+    __syncwarp();
+  }
 }
 
 __device__ __forceinline__ void group_bar(int g) {
@@ -263,7 +296,8 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_bf16_kernel(const __grid_const
       const long wrow0 = r0 + qd * 32;
       const int wrows = max(0, min(32, nrows - qd * 32));
       float al = 0.f;
-      if (EPI == EPI_EDGE && live) al = __ldg(a.pin + __ldg(a.src + grow)) + __ldg(a.qin + __ldg(a.dst + grow));
+      if ((EPI == EPI_EDGE || EPI == EPI_EDGEBWD) && live)
+        al = __ldg(a.pin + __ldg(a.src + grow)) + __ldg(a.qin + __ldg(a.dst + grow));
       tc::mbar_wait(accfull + j, (i / NG) & 1);
       tc::fence_after_sync();
       const uint32_t acc = lane_base + acc_col(j) + cb;
@@ -302,6 +336,49 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_bf16_kernel(const __grid_const
           for (int u = 0; u < 16; ++u) o[u] = fast_rcp(1.f + ex2(__uint_as_float(r[u]) * cexp));  // e' (R2, R3)
           warp_store_bf16(wbuf, a.out, wrow0, wrows, cb + c0, D, o, lane);
         }
+      } else if (EPI == EPI_EDGEBWD) {
+        const float cexp = al * LOG2E;
+        double dpart = 0.0;                       // dα = <dy, z> in float64 (cancellation)
+#pragma unroll 1
+        for (int c0 = 0; c0 < DH; c0 += 16) {
+          uint32_t r[16];
+          tc::tmem_ld16(acc + c0, r);
+          float ev[16], dv[16];
+          if (live) {
+            const uint4 *ep = reinterpret_cast<const uint4 *>(a.eb + grow * D + cb + c0);
+            const float4 *dp = reinterpret_cast<const float4 *>(a.de + grow * D + cb + c0);
+            const uint4 e0 = __ldg(ep), e1 = __ldg(ep + 1);
+            const uint32_t ew[8] = {e0.x, e0.y, e0.z, e0.w, e1.x, e1.y, e1.z, e1.w};
+#pragma unroll
+            for (int u = 0; u < 8; ++u) {
+              ev[2 * u] = __uint_as_float(ew[u] << 16);
+              ev[2 * u + 1] = __uint_as_float(ew[u] & 0xFFFF0000u);
+            }
+#pragma unroll
+            for (int u = 0; u < 4; ++u) {
+              const float4 x = __ldg(dp + u);
+              dv[4 * u] = x.x; dv[4 * u + 1] = x.y; dv[4 * u + 2] = x.z; dv[4 * u + 3] = x.w;
+            }
+          } else {
+#pragma unroll
+            for (int u = 0; u < 16; ++u) ev[u] = dv[u] = 0.f;
+          }
+          tc::tmem_ld_wait();
+          float o[16];
+#pragma unroll
+          for (int u = 0; u < 16; ++u) {
+            const float z = __uint_as_float(r[u]);
+            // σ'(y) = σ(y)·σ(-y): σ(y) is the stored e', σ(-y) from the recomputed y = α z
+            const float dy = dv[u] * ev[u] * fast_rcp(1.f + ex2(z * cexp));
+            dpart = fma(double(dy), double(z), dpart);
+            o[u] = al * dy;
+          }
+          warp_store_f32(reinterpret_cast<float *>(wbuf), a.outf, wrow0, wrows, cb + c0, D, o, lane);
+        }
+        double *xd = reinterpret_cast<double *>(xg);   // the group's exchange area
+        xd[hf * 128 + row] = dpart;
+        group_bar(g);
+        if (hf == 0 && live) a.dal[grow] = float(dpart + xd[128 + row]);
       } else {
         float m = 0.f;
         if (!noshift) {
@@ -518,7 +595,34 @@ int forward_layer_bf16(const occu_ctx *ctx, const DevCsr &csr, int layer, const 
   return n + r;
 }
 
+template <int D>
+int bwd_edge_bf16(const occu_ctx *ctx, const DevCsr &csr, int layer, const void *e_in, int Ke,
+                  const void *e, const float *de, const float *p, const float *q, float *DZ,
+                  float *dal, cudaStream_t st) {
+  BfArgs re{};
+  re.slope = ctx->cfg.slope;
+  re.rev = 0;
+  re.K = Ke; re.R = csr.E;
+  re.wimg = tc_wimg(ctx, 1, layer); re.wf = tc_wfexp(ctx, 1, layer);
+  re.pin = p; re.qin = q; re.src = csr.in_src; re.dst = csr.in_dst;
+  re.eb = reinterpret_cast<const __nv_bfloat16 *>(e);
+  re.de = de; re.outf = DZ; re.dal = dal;
+  return launch_bf<D, EPI_EDGEBWD, false>(ctx, re, e_in, "edge_bwd_tc", st);
+}
+
 }  // namespace
+
+int launch_bwd_edge_bf16(const occu_ctx *ctx, const DevCsr &csr, int layer, const void *e_in,
+                         int Ke, const void *e, const float *de, const float *p, const float *q,
+                         float *DZ, float *dal, cudaStream_t st) {
+  if (csr.E <= 0) return 0;
+  if (Ke != ctx->cfg.d) return -int(cudaErrorInvalidValue);
+  switch (ctx->cfg.d) {
+    case 64: return bwd_edge_bf16<64>(ctx, csr, layer, e_in, Ke, e, de, p, q, DZ, dal, st);
+    case 128: return bwd_edge_bf16<128>(ctx, csr, layer, e_in, Ke, e, de, p, q, DZ, dal, st);
+    default: return -int(cudaErrorInvalidValue);
+  }
+}
 
 int launch_forward_layer_bf16(const occu_ctx *ctx, const DevCsr &csr, int layer,
                               const FwdLayerArgs &a, cudaStream_t st) {

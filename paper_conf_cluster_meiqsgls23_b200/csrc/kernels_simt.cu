@@ -17,6 +17,7 @@
 #include <stdint.h>
 
 #include <algorithm>
+#include <cstdlib>
 
 #include "occu_internal.h"
 
@@ -29,6 +30,13 @@ constexpr int NT = 256;
 __device__ __forceinline__ float lrelu(float x, float s) { return x > 0.f ? x : s * x; }
 __device__ __forceinline__ float lrelu_grad_from_out(float y, float s) { return y > 0.f ? 1.f : s; }
 __device__ __forceinline__ float sigmoidf_(float x) { return 1.f / (1.f + expf(-x)); }
+// Element i of an FP32 or (BF = true) BF16 stored activation (OCCU_BF16 training, R28).
+template <bool BF> __device__ __forceinline__ float ld_act(const void *base, long i) {
+  if constexpr (BF)
+    return __uint_as_float(uint32_t(__ldg(reinterpret_cast<const unsigned short *>(base) + i)) << 16);
+  else
+    return __ldg(reinterpret_cast<const float *>(base) + i);
+}
 
 __device__ __forceinline__ float hsum16(float v) {   // sum over the 16 lanes sharing ty
   v += __shfl_xor_sync(0xffffffffu, v, 1);
@@ -609,9 +617,9 @@ __global__ void __launch_bounds__(NT, (BF ? G <= 8 : G == 4) ? 4 : 3) gather_seg
 // A warp takes 32 consecutive in-CSR edges, four at a time with all row loads of the
 // four in flight; lane = D/32 channels; the dot is a fixed-order butterfly.
 // ---------------------------------------------------------------------------
-template <int D>
+template <int D, bool BF>
 __global__ void __launch_bounds__(NT) gate_bwd_stream_kernel(
-    const float *__restrict__ g, const float *__restrict__ dA, const float *__restrict__ hbar,
+    const void *__restrict__ g, const float *__restrict__ dA, const void *__restrict__ hbar,
     const int32_t *__restrict__ in_src, const int32_t *__restrict__ in_dst, int E,
     float *__restrict__ MG, float *__restrict__ DV) {
   constexpr int V = D / 32;
@@ -623,7 +631,8 @@ __global__ void __launch_bounds__(NT) gate_bwd_stream_kernel(
     const int s_l = lane < cnt ? __ldg(in_src + k0 + lane) : 0;
     const int t_l = lane < cnt ? __ldg(in_dst + k0 + lane) : 0;
     for (int j = 0; j < cnt; j += G) {
-      RawRow<V, false> gr[G], dr[G], hr[G];
+      RawRow<V, BF> gr[G], hr[G];
+      RawRow<V, false> dr[G];
 #pragma unroll
       for (int u = 0; u < G; ++u) {
         const int kk = min(j + u, cnt - 1);
@@ -833,7 +842,8 @@ __global__ void head_bwd_reduce_kernel(const float *__restrict__ dy, const float
 // h_mask != null: emit dA = dh ⊙ LReLU'(A) (÷ deg for MEAN; sign(A) = sign(h)) instead of dh.
 __global__ void broadcast_dh_kernel(const float *__restrict__ dr, const int32_t *__restrict__ node_graph,
                                     const int32_t *__restrict__ node_off, int N, int D,
-                                    const float *__restrict__ h_mask, const int32_t *__restrict__ in_ptr,
+                                    const void *__restrict__ h_mask, int mask_bf,
+                                    const int32_t *__restrict__ in_ptr,
                                     int mean, float slope, float *__restrict__ dh) {
   const long total = long(N) * D;
   for (long i = blockIdx.x * long(blockDim.x) + threadIdx.x; i < total;
@@ -842,7 +852,7 @@ __global__ void broadcast_dh_kernel(const float *__restrict__ dr, const int32_t 
     const int b = node_graph[u];
     float v = dr[long(b) * D + k] / float(node_off[b + 1] - node_off[b]);
     if (h_mask) {
-      v = v * lrelu_grad_from_out(h_mask[i], slope);
+      v = v * lrelu_grad_from_out(mask_bf ? ld_act<true>(h_mask, i) : ld_act<false>(h_mask, i), slope);
       if (mean) {
         const int deg = in_ptr[u + 1] - in_ptr[u];
         v = v / float(deg > 0 ? deg : 1);
@@ -960,9 +970,9 @@ __global__ void __launch_bounds__(NT) edge_bwd_m_kernel(
 
 // Edge backward, phase B (W_e): dy = de ⊙ e'(1-e') ; z = W_e e_in (recompute) ;
 // dα = <dy, z> ; dz = α dy ; de_prev = W_eᵀ dz (layer > 0).
-template <int D>
+template <int D, bool BF>
 __global__ void __launch_bounds__(NT) edge_bwd_e_kernel(
-    const float *__restrict__ e_in, int Ke, const float *__restrict__ e, const float *__restrict__ de,
+    const float *__restrict__ e_in, int Ke, const void *__restrict__ e, const float *__restrict__ de,
     const float *__restrict__ W_e, const float *__restrict__ p, const float *__restrict__ q,
     const int32_t *__restrict__ in_src, const int32_t *__restrict__ in_dst, int E,
     float *__restrict__ DZ, float *__restrict__ dalpha, float *__restrict__ de_prev) {
@@ -999,7 +1009,12 @@ __global__ void __launch_bounds__(NT) edge_bwd_e_kernel(
       float ev[TN], dev[TN];
       double dad = 0.0;
       if (r < nrows) {
-        load_row<D>(e + (k0 + r) * D, ev, tx);
+        if constexpr (BF) {
+#pragma unroll
+          for (int j = 0; j < TN; ++j) ev[j] = ld_act<true>(e, (k0 + r) * D + colof<D>(tx, j));
+        } else {
+          load_row<D>(reinterpret_cast<const float *>(e) + (k0 + r) * D, ev, tx);
+        }
         load_row<D>(de + (k0 + r) * D, dev, tx);
       } else {
 #pragma unroll
@@ -1039,10 +1054,10 @@ __global__ void __launch_bounds__(NT) edge_bwd_e_kernel(
 // Node backward (warp per node u):
 //   dh̄_u = Σ_{out-edges} MG + dp_u a_s + dq_u a_d ; dP = dh̄ ⊙ LReLU'(h̄)
 //   dp_u = Σ_{out-edges} dα ; dq_u = Σ_{in-edges} dα
-template <int D>
+template <int D, bool BF>
 __global__ void __launch_bounds__(NT) node_bwd_kernel(
     const float *__restrict__ MG, const float *__restrict__ dalpha,
-    const float *__restrict__ hbar, const float *__restrict__ a_s, const float *__restrict__ a_d,
+    const void *__restrict__ hbar, const float *__restrict__ a_s, const float *__restrict__ a_d,
     const int32_t *__restrict__ out_ptr, const int32_t *__restrict__ out_pos,
     const int32_t *__restrict__ in_ptr, int N, float slope, float *__restrict__ dP,
     float *__restrict__ dpq, float *__restrict__ da_part) {
@@ -1072,7 +1087,7 @@ __global__ void __launch_bounds__(NT) node_bwd_kernel(
     for (int c = 0; c < V; ++c) {
       const int ch = lane * V + c;
       const float v = acc[c] + dp * a_s[ch] + dq * a_d[ch];
-      const float hb = hbar[long(u) * D + ch];
+      const float hb = ld_act<BF>(hbar, long(u) * D + ch);
       dP[long(u) * D + ch] = v * lrelu_grad_from_out(hb, slope);
       das[c] = fmaf(dp, hb, das[c]);
       dad[c] = fmaf(dq, hb, dad[c]);
@@ -1438,8 +1453,10 @@ static int reduce_splits(const occu_ctx *ctx, const float *part, int splits, lon
   return 1;
 }
 
-static int wgrad(occu_ctx *ctx, const float *X, int A, const float *Y, int Bn, long R, float *out,
-                 cudaStream_t st) {
+// ybf: Y holds BF16 rows (OCCU_BF16 training); only the tensor-core kernel reads those.
+static int wgrad(occu_ctx *ctx, const float *X, int A, const void *Yv, int Bn, long R, float *out,
+                 cudaStream_t st, bool ybf = false) {
+  const float *Y = reinterpret_cast<const float *>(Yv);
   const long n = long(A) * Bn;
   const int ta = (A + 127) / 128, tb = (Bn + 127) / 128;
   int splits = int(std::max<long>(1, std::min<long>((2L * ctx->num_sms) / (ta * tb), (R + 255) / 256)));
@@ -1447,11 +1464,13 @@ static int wgrad(occu_ctx *ctx, const float *X, int A, const float *Y, int Bn, l
     cudaMemsetAsync(out, 0, n * 4, st);
     return 0;
   }
-  if (ctx->path != 1 && wgrad_tc_supported(A, Bn) && R >= 4096) {
+  if (ybf && !wgrad_tc_supported(A, Bn)) return -int(cudaErrorInvalidValue);
+  static const long tc_min = getenv("OCCU_WGRAD_TC_MIN") ? atol(getenv("OCCU_WGRAD_TC_MIN")) : 4096;
+  if (ctx->path != 1 && wgrad_tc_supported(A, Bn) && (R >= tc_min || ybf)) {
     const int sp = ctx->num_sms;
     if (ctx->ws.partial.ensure(size_t(sp) * n * 4) != cudaSuccess) return -int(cudaErrorMemoryAllocation);
     float *part = ctx->ws.partial.as<float>();
-    int r = launch_wgrad_tc(ctx, X, A, Y, Bn, R, sp, part, st);
+    int r = launch_wgrad_tc(ctx, X, A, Yv, Bn, R, sp, part, st, ybf);
     if (r < 0) return r;
     return r + reduce_splits(ctx, part, sp, n, out, st);
   }
@@ -1476,6 +1495,11 @@ static int wgrad(occu_ctx *ctx, const float *X, int A, const float *Y, int Bn, l
   OCCU_PROF_END(ctx);
   LAUNCH_CHECK();
   return 2;
+}
+
+int launch_wgrad(occu_ctx *ctx, const float *X, int A, const void *Y, int Bn, long R, float *out,
+                 cudaStream_t st, bool ybf) {
+  return wgrad(ctx, X, A, Y, Bn, R, out, st, ybf);
 }
 
 int launch_head_backward(occu_ctx *ctx, const DevCsr &csr, const float *targets, int global_B,
@@ -1504,7 +1528,8 @@ int launch_head_backward(occu_ctx *ctx, const DevCsr &csr, const float *targets,
   const bool tcb = ctx->path != 1 && tc_supported(cf);    // TC backward consumes dA directly
   broadcast_dh_kernel<<<grid_for(long(csr.N) * cf.d, 256, 8192), 256, 0, st>>>(
       w.dr.as<float>(), csr.node_graph, csr.node_off, csr.N, cf.d,
-      tcb ? w.h[cf.L - 1].as<float>() : nullptr, csr.in_ptr, cf.aggr == OCCU_AGGR_MEAN, cf.slope,
+      tcb ? w.h[cf.L - 1].ptr : nullptr, cf.prec == OCCU_BF16 ? 1 : 0, csr.in_ptr,
+      cf.aggr == OCCU_AGGR_MEAN, cf.slope,
       w.dh.as<float>());
   OCCU_PROF_END(ctx);
   LAUNCH_CHECK();
@@ -1524,14 +1549,21 @@ static int backward_layer_impl(occu_ctx *ctx, const DevCsr &csr, const BwdLayerA
   int n = 0;
   float *de = w.deA.as<float>();
   const bool tc = ctx->path != 1 && tc_supported(cf);
+  const bool bf = a.bf;                     // OCCU_BF16: stored activations are BF16 (R28)
+  const bool in_bf = bf && i > 0;           // h_in, e_in of layer 1 are the FP32 inputs
+  if (bf && !(tc && a.g)) return -int(cudaErrorInvalidValue);
   int r;
   if (tc && csr.E > 0) {
     // a10: softmax / message backward (streaming with the saved gates, else g recomputed on
     // tensor cores), W_mᵀ dv, z recompute + σ', W_eᵀ dz on tensor cores
     if (a.g) {
       OCCU_PROF_BEGIN(ctx, "gate_bwd", st);
-      gate_bwd_stream_kernel<D><<<grid_for((long(csr.E) + 31) / 32, NT / 32, 8 * sms), NT, 0, st>>>(
-          a.g, a.dh, a.hbar, csr.in_src, csr.in_dst, csr.E, w.MG.as<float>(), w.DV.as<float>());
+      if (bf)
+        gate_bwd_stream_kernel<D, true><<<grid_for((long(csr.E) + 31) / 32, NT / 32, 8 * sms), NT, 0, st>>>(
+            a.g, a.dh, a.hbar, csr.in_src, csr.in_dst, csr.E, w.MG.as<float>(), w.DV.as<float>());
+      else
+        gate_bwd_stream_kernel<D, false><<<grid_for((long(csr.E) + 31) / 32, NT / 32, 8 * sms), NT, 0, st>>>(
+            a.g, a.dh, a.hbar, csr.in_src, csr.in_dst, csr.E, w.MG.as<float>(), w.DV.as<float>());
       OCCU_PROF_END(ctx);
       LAUNCH_CHECK();
       ++n;
@@ -1543,7 +1575,11 @@ static int backward_layer_impl(occu_ctx *ctx, const DevCsr &csr, const BwdLayerA
     if ((r = launch_plain_tc(ctx, w.DV.as<float>(), D, csr.E, 3, i, a.de_out, de,
                              "de_tc", st)) < 0) return r;
     n += r;
-    if (a.Ke > 16) {
+    if (a.Ke > 16 && bf) {
+      if ((r = launch_bwd_edge_bf16(ctx, csr, i, a.e_in, a.Ke, a.e, de, a.p, a.q,
+                                    w.DZ.as<float>(), w.dalpha.as<float>(), st)) < 0) return r;
+      n += r;
+    } else if (a.Ke > 16) {
       if ((r = launch_bwd_edge_tc(ctx, csr, i, a.e_in, a.Ke, a.e, de, a.p, a.q,
                                   w.DZ.as<float>(), w.dalpha.as<float>(), st)) < 0) return r;
       n += r;
@@ -1551,11 +1587,18 @@ static int backward_layer_impl(occu_ctx *ctx, const DevCsr &csr, const BwdLayerA
       const int tiles = (csr.E + BM - 1) / BM;
       const int KS = a.Ke > D ? a.Ke : D;
       const size_t smB = (size_t(a.Ke) * D + BM * (KS + 4) + BM) * 4;
-      set_smem(edge_bwd_e_kernel<D>, smB);
       OCCU_PROF_BEGIN(ctx, "edge_bwd_e", st);
-      edge_bwd_e_kernel<D><<<grid_for(tiles, 1, sms), NT, smB, st>>>(
-          a.e_in, a.Ke, a.e, de, P + L.W_e[i], a.p, a.q, csr.in_src, csr.in_dst, csr.E,
-          w.DZ.as<float>(), w.dalpha.as<float>(), nullptr);
+      if (bf) {    // layer 1 only (Ke <= 16): e_in is the FP32 e0, e' is BF16
+        set_smem(edge_bwd_e_kernel<D, true>, smB);
+        edge_bwd_e_kernel<D, true><<<grid_for(tiles, 1, sms), NT, smB, st>>>(
+            a.e_in, a.Ke, a.e, de, P + L.W_e[i], a.p, a.q, csr.in_src, csr.in_dst, csr.E,
+            w.DZ.as<float>(), w.dalpha.as<float>(), nullptr);
+      } else {
+        set_smem(edge_bwd_e_kernel<D, false>, smB);
+        edge_bwd_e_kernel<D, false><<<grid_for(tiles, 1, sms), NT, smB, st>>>(
+            a.e_in, a.Ke, a.e, de, P + L.W_e[i], a.p, a.q, csr.in_src, csr.in_dst, csr.E,
+            w.DZ.as<float>(), w.dalpha.as<float>(), nullptr);
+      }
       OCCU_PROF_END(ctx);
       LAUNCH_CHECK();
       ++n;
@@ -1578,9 +1621,9 @@ static int backward_layer_impl(occu_ctx *ctx, const DevCsr &csr, const BwdLayerA
     ++n;
     const int KS = a.Ke > D ? a.Ke : D;
     const size_t smB = (size_t(a.Ke) * D + (a.de_prev ? D * a.Ke : 0) + BM * (KS + 4) + BM) * 4;
-    set_smem(edge_bwd_e_kernel<D>, smB);
+    set_smem(edge_bwd_e_kernel<D, false>, smB);
     OCCU_PROF_BEGIN(ctx, "edge_bwd_e", st);
-    edge_bwd_e_kernel<D><<<grid_for(tiles, 1, sms), NT, smB, st>>>(
+    edge_bwd_e_kernel<D, false><<<grid_for(tiles, 1, sms), NT, smB, st>>>(
         a.e_in, a.Ke, a.e, de, P + L.W_e[i], a.p, a.q, csr.in_src, csr.in_dst, csr.E,
         w.DZ.as<float>(), w.dalpha.as<float>(), a.de_prev);
     OCCU_PROF_END(ctx);
@@ -1594,9 +1637,14 @@ static int backward_layer_impl(occu_ctx *ctx, const DevCsr &csr, const BwdLayerA
     da_part = w.dpart.as<float>();
   }
   OCCU_PROF_BEGIN(ctx, "node_bwd", st);
-  node_bwd_kernel<D><<<nb_blocks, NT, 0, st>>>(
-      w.MG.as<float>(), w.dalpha.as<float>(), a.hbar, P + L.a_s[i], P + L.a_d[i], csr.out_ptr,
-      csr.out_pos, csr.in_ptr, csr.N, cf.slope, w.dP.as<float>(), w.dpq.as<float>(), da_part);
+  if (bf)
+    node_bwd_kernel<D, true><<<nb_blocks, NT, 0, st>>>(
+        w.MG.as<float>(), w.dalpha.as<float>(), a.hbar, P + L.a_s[i], P + L.a_d[i], csr.out_ptr,
+        csr.out_pos, csr.in_ptr, csr.N, cf.slope, w.dP.as<float>(), w.dpq.as<float>(), da_part);
+  else
+    node_bwd_kernel<D, false><<<nb_blocks, NT, 0, st>>>(
+        w.MG.as<float>(), w.dalpha.as<float>(), a.hbar, P + L.a_s[i], P + L.a_d[i], csr.out_ptr,
+        csr.out_pos, csr.in_ptr, csr.N, cf.slope, w.dP.as<float>(), w.dpq.as<float>(), da_part);
   OCCU_PROF_END(ctx);
   LAUNCH_CHECK();
   ++n;
@@ -1605,11 +1653,11 @@ static int backward_layer_impl(occu_ctx *ctx, const DevCsr &csr, const BwdLayerA
     n += r;
   }
   // dW_m = DVᵀ E' ; dW_e = DZᵀ E_in ; dW_u = dPᵀ H_in ; [da_s; da_d] = [dp dq]ᵀ h̄
-  if ((r = wgrad(ctx, w.DV.as<float>(), D, a.e, D, csr.E, G + L.W_m[i], st)) < 0) return r;
+  if ((r = wgrad(ctx, w.DV.as<float>(), D, a.e, D, csr.E, G + L.W_m[i], st, bf)) < 0) return r;
   n += r;
-  if ((r = wgrad(ctx, w.DZ.as<float>(), D, a.e_in, a.Ke, csr.E, G + L.W_e[i], st)) < 0) return r;
+  if ((r = wgrad(ctx, w.DZ.as<float>(), D, a.e_in, a.Ke, csr.E, G + L.W_e[i], st, in_bf)) < 0) return r;
   n += r;
-  if ((r = wgrad(ctx, w.dP.as<float>(), D, a.h_in, a.K, csr.N, G + L.W_u[i], st)) < 0) return r;
+  if ((r = wgrad(ctx, w.dP.as<float>(), D, a.h_in, a.K, csr.N, G + L.W_u[i], st, in_bf)) < 0) return r;
   n += r;
   if (!tc) {
     if ((r = wgrad(ctx, w.dpq.as<float>(), 2, a.hbar, D, csr.N, G + L.a_s[i], st)) < 0) return r;
@@ -1617,7 +1665,7 @@ static int backward_layer_impl(occu_ctx *ctx, const DevCsr &csr, const BwdLayerA
   }
   if (a.dh_prev && csr.N > 0 && tc) {   // dh^{i-1} = dP W_u on tensor cores
     if ((r = launch_plain_tc(ctx, w.dP.as<float>(), D, csr.N, 5, i, nullptr, a.dh_prev,
-                             "dh_prev_tc", st, a.h_in, csr.in_ptr)) < 0) return r;
+                             "dh_prev_tc", st, a.h_in, csr.in_ptr, in_bf)) < 0) return r;
     n += r;
   } else if (a.dh_prev && csr.N > 0) {   // dh^{i-1} = dP W_u  (K == D for i > 0)
     const size_t sm1 = (size_t(D) * D + BM * (D + 4)) * 4;

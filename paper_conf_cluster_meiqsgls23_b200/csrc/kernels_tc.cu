@@ -119,6 +119,7 @@ struct RowGemmArgs {
   float *out2;             // GATEBWD: DV
   const float *dh, *h, *hbar, *e, *de;
   const float *mask_h;     // PLAIN: multiply row by LReLU'(mask_h row) (÷ deg for MEAN) -> dA
+  int mask_bf;             // mask_h rows are BF16 (OCCU_BF16 training)
   const int32_t *in_ptr;
   int mean;
   float *dal;              // EDGEBWD: dα [R]
@@ -462,6 +463,7 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
           for (int u = 0; u < 16; ++u) o[u] = __uint_as_float(r[u]) * un;
           if (a.mask_h && live) {
             const float *mr = a.mask_h + grow * D + cb + c0;
+            const uint16_t *mb = reinterpret_cast<const uint16_t *>(a.mask_h) + grow * D + cb + c0;
             float dsc = 1.f;
             if (a.mean) {
               const int deg = __ldg(a.in_ptr + grow + 1) - __ldg(a.in_ptr + grow);
@@ -469,7 +471,14 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
             }
 #pragma unroll
             for (int u = 0; u < 16; u += 4) {
-              const float4 x = __ldg(reinterpret_cast<const float4 *>(mr + u));
+              float4 x;
+              if (a.mask_bf) {      // only the sign matters: BF16 keeps it
+                const uint2 b = __ldg(reinterpret_cast<const uint2 *>(mb + u));
+                x = make_float4(__uint_as_float(b.x << 16), __uint_as_float(b.x & 0xFFFF0000u),
+                                __uint_as_float(b.y << 16), __uint_as_float(b.y & 0xFFFF0000u));
+              } else {
+                x = __ldg(reinterpret_cast<const float4 *>(mr + u));
+              }
               const float xv[4] = {x.x, x.y, x.z, x.w};
 #pragma unroll
               for (int t = 0; t < 4; ++t) {
@@ -1347,9 +1356,19 @@ __global__ void __launch_bounds__(256) edge_small_kernel(
 // SW128 boxes) and are consumed as MN-major operands (M = a, N = b, K = row).  Each CTA
 // owns a contiguous row range; partials are reduced in fixed split order afterwards.
 // ---------------------------------------------------------------------------
+// YBF (OCCU_BF16 training, R28): Y rows are BF16.  TMA lands them (32 rows x 64 bf16 SW128
+// boxes) in the Y-lo region; the lo warps widen them (exactly) into the Y raw region, and
+// since a BF16 value is its own tf32 hi part (Y lo = 0) the X_hi·Y_lo product is skipped.
 constexpr int WG_NS = 3;                  // pipeline stages of 32 rows
 constexpr int WG_NTH = 320;               // warp0 TMA, warp1 MMA, warps 2-9 lo / epilogue
 
+// Logical 16-byte chunk stored at physical slot pc of 128-byte row r under the TMA
+// SWIZZLE_128B_ATOM_32B pattern (32-byte chunks permuted: chunk32 ^ (r & 3)).
+__device__ __forceinline__ int wg_logical_chunk(int pc, int r) {
+  return ((((pc >> 1) ^ (r & 3))) << 1) | (pc & 1);
+}
+
+template <bool YBF>
 __global__ void __launch_bounds__(WG_NTH, 1)
 wgrad_tc_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant__ CUtensorMap ymap,
                 int A, int Bn, long R, int splits, float *__restrict__ partial) {
@@ -1362,7 +1381,7 @@ wgrad_tc_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant_
   uint64_t *full = bars, *lo_ready = bars + WG_NS, *empty = bars + 2 * WG_NS, *done = bars + 3 * WG_NS;
   uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(bars + 3 * WG_NS + 1);
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const int nbx = (A + 31) / 32, nby = (Bn + 31) / 32;
+  const int nbx = (A + 31) / 32, nby = (Bn + 31) / 32, nbyb = (Bn + 63) / 64;
   const int Npad = (Bn + 15) / 16 * 16;
   // zero every box region once: boxes that TMA never writes (A or B < 128) stay zero
   for (int i = threadIdx.x; i < WG_NS * 65536 / 16; i += WG_NTH)
@@ -1395,9 +1414,12 @@ wgrad_tc_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant_
         if (i >= WG_NS) tc::mbar_wait(empty + j, ((i / WG_NS) - 1) & 1);
         const int r0 = int(rb + long(i) * 32);
         uint8_t *st = stage(j);
-        tc::mbar_arrive_expect_tx(full + j, uint32_t(nbx + nby) * 4096u);
+        tc::mbar_arrive_expect_tx(full + j, uint32_t(nbx + (YBF ? nbyb : nby)) * 4096u);
         for (int b = 0; b < nbx; ++b) tc::tma_load_2d(st + b * 4096, &xmap, 32 * b, r0, full + j);
-        for (int b = 0; b < nby; ++b) tc::tma_load_2d(st + 32768 + b * 4096, &ymap, 32 * b, r0, full + j);
+        if (YBF)
+          for (int b = 0; b < nbyb; ++b) tc::tma_load_2d(st + 49152 + b * 4096, &ymap, 64 * b, r0, full + j);
+        else
+          for (int b = 0; b < nby; ++b) tc::tma_load_2d(st + 32768 + b * 4096, &ymap, 32 * b, r0, full + j);
       }
     }
     __syncwarp();
@@ -1410,12 +1432,12 @@ wgrad_tc_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant_
       if (lane == 0) {
         const uint32_t st = tc::smem_u32(stage(j));
         for (int kg = 0; kg < 4; ++kg) {
-          const uint64_t ah = tc::sdesc_sw128_mn(st + kg * 1024, 4096);
-          const uint64_t al = tc::sdesc_sw128_mn(st + 16384 + kg * 1024, 4096);
-          const uint64_t bh = tc::sdesc_sw128_mn(st + 32768 + kg * 1024, 4096);
-          const uint64_t bl = tc::sdesc_sw128_mn(st + 49152 + kg * 1024, 4096);
+          const uint64_t ah = tc::sdesc_sw128b32_mn(st + kg * 1024, 4096);
+          const uint64_t al = tc::sdesc_sw128b32_mn(st + 16384 + kg * 1024, 4096);
+          const uint64_t bh = tc::sdesc_sw128b32_mn(st + 32768 + kg * 1024, 4096);
+          const uint64_t bl = tc::sdesc_sw128b32_mn(st + 49152 + kg * 1024, 4096);
           tc::mma_tf32_ss(tmem, ah, bh, idsc, (i > 0 || kg > 0) ? 1u : 0u);
-          tc::mma_tf32_ss(tmem, ah, bl, idsc, 1u);
+          if (!YBF) tc::mma_tf32_ss(tmem, ah, bl, idsc, 1u);
           tc::mma_tf32_ss(tmem, al, bh, idsc, 1u);
         }
         tc::mma_commit(empty + j);
@@ -1437,14 +1459,31 @@ wgrad_tc_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant_
       for (int it = 0; it < 8; ++it) {
         const int f = t + it * 256, op = f >> 10, b = (f >> 8) & 3, q4 = f & 255;
         v[it] = make_float4(0.f, 0.f, 0.f, 0.f);
-        if (b < (op == 0 ? nbx : nby))
-          v[it] = reinterpret_cast<const float4 *>(st + op * 32768 + b * 4096)[q4];
+        if (b < (op == 0 ? nbx : nby)) {
+          if (YBF && op == 1) {
+            // fp32 box b (SWIZZLE_128B_ATOM_32B), row rr, physical 16-byte slot q4 & 7 holds
+            // logical chunk c (columns 32b+4c..+3) <- bf16 box b/2 (plain SW128: chunk ^ (row & 7)),
+            // logical chunk 4(b&1) + c/2, half c&1
+            const int rr = q4 >> 3, c = wg_logical_chunk(q4 & 7, rr), cb = 4 * (b & 1) + (c >> 1);
+            const uint2 w = *reinterpret_cast<const uint2 *>(st + 49152 + (b >> 1) * 4096 + rr * 128 +
+                                                             ((cb ^ (rr & 7)) << 4) + (c & 1) * 8);
+            v[it] = make_float4(__uint_as_float(w.x << 16), __uint_as_float(w.x & 0xFFFF0000u),
+                                __uint_as_float(w.y << 16), __uint_as_float(w.y & 0xFFFF0000u));
+          } else {
+            v[it] = reinterpret_cast<const float4 *>(st + op * 32768 + b * 4096)[q4];
+          }
+        }
       }
 #pragma unroll
       for (int it = 0; it < 8; ++it) {
         const int f = t + it * 256, op = f >> 10, b = (f >> 8) & 3, q4 = f & 255;
         if (b >= (op == 0 ? nbx : nby)) continue;
         float4 x = v[it];
+        if (YBF && op == 1) {                             // widened BF16 row: raw, no lo
+          if (r0 + (q4 >> 3) >= re) x = make_float4(0.f, 0.f, 0.f, 0.f);
+          reinterpret_cast<float4 *>(st + 32768 + b * 4096)[q4] = x;
+          continue;
+        }
         if (r0 + (q4 >> 3) >= re) {                       // 8 float4 per 128-byte row
           x = make_float4(0.f, 0.f, 0.f, 0.f);
           reinterpret_cast<float4 *>(st + op * 32768 + b * 4096)[q4] = x;
@@ -1577,6 +1616,26 @@ static bool encode_rows_map32(CUtensorMap *m, const float *A, long R, int K) {
   const cuuint32_t box[2] = {32, 32};
   const cuuint32_t estr[2] = {1, 1};
   return fn(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, const_cast<float *>(A), dims, strides, box, estr,
+            CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B,
+            CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
+// BF16 rows [R][K]: boxes of 32 rows x 64 bf16 (128 B), 128-byte swizzle, OOB zero.
+static bool encode_rows_map32_bf16(CUtensorMap *m, const void *A, long R, int K) {
+  static PFN_encodeTiled fn = nullptr;
+  if (!fn) {
+    void *p = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) != cudaSuccess ||
+        q != cudaDriverEntryPointSuccess || !p)
+      return false;
+    fn = reinterpret_cast<PFN_encodeTiled>(p);
+  }
+  const cuuint64_t dims[2] = {cuuint64_t(K), cuuint64_t(R)};
+  const cuuint64_t strides[1] = {cuuint64_t(K) * 2};
+  const cuuint32_t box[2] = {64, 32};
+  const cuuint32_t estr[2] = {1, 1};
+  return fn(m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void *>(A), dims, strides, box, estr,
             CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
             CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
@@ -1586,15 +1645,21 @@ bool wgrad_tc_supported(int A, int Bn) {
 }
 
 // partial must hold splits * A * Bn floats; returns the number of launches (1) or -err.
-int launch_wgrad_tc(const occu_ctx *ctx, const float *X, int A, const float *Y, int Bn, long R,
-                    int splits, float *partial, cudaStream_t st) {
+int launch_wgrad_tc(const occu_ctx *ctx, const float *X, int A, const void *Y, int Bn, long R,
+                    int splits, float *partial, cudaStream_t st, bool ybf) {
   CUtensorMap xm, ym;
-  if (!encode_rows_map32(&xm, X, R, A) || !encode_rows_map32(&ym, Y, R, Bn))
+  if (!encode_rows_map32(&xm, X, R, A) ||
+      !(ybf ? encode_rows_map32_bf16(&ym, Y, R, Bn) : encode_rows_map32(&ym, static_cast<const float *>(Y), R, Bn)))
     return -int(cudaErrorInvalidValue);
   const size_t smem = 1024 + WG_NS * 65536 + 256;
-  set_smem(wgrad_tc_kernel, smem);
   OCCU_PROF_BEGIN(ctx, "wgrad_tc", st);
-  wgrad_tc_kernel<<<splits, WG_NTH, smem, st>>>(xm, ym, A, Bn, R, splits, partial);
+  if (ybf) {
+    set_smem(wgrad_tc_kernel<true>, smem);
+    wgrad_tc_kernel<true><<<splits, WG_NTH, smem, st>>>(xm, ym, A, Bn, R, splits, partial);
+  } else {
+    set_smem(wgrad_tc_kernel<false>, smem);
+    wgrad_tc_kernel<false><<<splits, WG_NTH, smem, st>>>(xm, ym, A, Bn, R, splits, partial);
+  }
   OCCU_PROF_END(ctx);
   TC_CHECK();
   return 1;
@@ -1624,7 +1689,9 @@ int tc_prepare_weights(occu_ctx *ctx, cudaStream_t st) {
     auto add = [&](int kind, const float *W, int D, int K, int transW) {
       WImageJob j;
       j.W = W; j.D = D; j.K = K; j.transW = transW;
-      j.bf16 = c.prec == OCCU_BF16;
+      // OCCU_BF16: the forward images (kinds 0-2) are BF16; the backward images (3-5) multiply
+      // FP32 gradients and stay fp16x2 FP32 images (R28)
+      j.bf16 = c.prec == OCCU_BF16 && kind <= 2;
       j.img = const_cast<uint8_t *>(tc_wimg(ctx, kind, i));
       j.fexp = const_cast<int *>(tc_wfexp(ctx, kind, i));
       jobs.push_back(j);
@@ -1815,8 +1882,9 @@ static int bwd_gate_impl(const occu_ctx *ctx, const DevCsr &csr, int layer, cons
 template <int D>
 static int plain_impl(const occu_ctx *ctx, const float *A, int K, int R, int wkind, int layer,
                       const float *add, float *out, const char *name, cudaStream_t st,
-                      const float *mask_h, const int32_t *in_ptr) {
+                      const float *mask_h, const int32_t *in_ptr, bool mask_bf) {
   RowGemmArgs r{};
+  r.mask_bf = mask_bf ? 1 : 0;
   r.slope = ctx->cfg.slope;
   r.A = A; r.K = K; r.R = R; r.add = add; r.out = out;
   r.wimg = tc_wimg(ctx, wkind, layer); r.wfexp = tc_wfexp(ctx, wkind, layer);
@@ -1844,10 +1912,10 @@ int launch_bwd_gate_tc(const occu_ctx *ctx, const DevCsr &csr, int layer, const 
 }
 int launch_plain_tc(const occu_ctx *ctx, const float *A, int K, int R, int wkind, int layer,
                     const float *add, float *out, const char *name, cudaStream_t st,
-                    const float *mask_h, const int32_t *in_ptr) {
+                    const float *mask_h, const int32_t *in_ptr, bool mask_bf) {
   if (R <= 0) return 0;
-  return ctx->cfg.d == 64 ? plain_impl<64>(ctx, A, K, R, wkind, layer, add, out, name, st, mask_h, in_ptr)
-                          : plain_impl<128>(ctx, A, K, R, wkind, layer, add, out, name, st, mask_h, in_ptr);
+  return ctx->cfg.d == 64 ? plain_impl<64>(ctx, A, K, R, wkind, layer, add, out, name, st, mask_h, in_ptr, mask_bf)
+                          : plain_impl<128>(ctx, A, K, R, wkind, layer, add, out, name, st, mask_h, in_ptr, mask_bf);
 }
 int launch_bwd_edge_tc(const occu_ctx *ctx, const DevCsr &csr, int layer, const float *e_in, int Ke,
                        const float *e, const float *de, const float *p, const float *q, float *DZ,

@@ -173,12 +173,18 @@ int launch_bwd_gate_tc(const occu_ctx *ctx, const DevCsr &csr, int layer, const 
                        cudaStream_t st);
 int launch_plain_tc(const occu_ctx *ctx, const float *A, int K, int R, int wkind, int layer,
                     const float *add, float *out, const char *name, cudaStream_t st,
-                    const float *mask_h = nullptr, const int32_t *in_ptr = nullptr);
+                    const float *mask_h = nullptr, const int32_t *in_ptr = nullptr,
+                    bool mask_bf = false);
+// OCCU_BF16 training: z = W_e e_in recomputed from BF16 e_in on the BF16 tensor-core path
+// (as the forward), epilogue dy = de ⊙ e' ⊙ σ(-αz) with BF16 e', dα = <dy, z>, DZ = α dy.
+int launch_bwd_edge_bf16(const occu_ctx *ctx, const DevCsr &csr, int layer, const void *e_in,
+                         int Ke, const void *e, const float *de, const float *p, const float *q,
+                         float *DZ, float *dal, cudaStream_t st);
 int launch_bwd_edge_tc(const occu_ctx *ctx, const DevCsr &csr, int layer, const float *e_in, int Ke,
                        const float *e, const float *de, const float *p,
                        const float *q, float *DZ, float *dal, cudaStream_t st);
-int launch_wgrad_tc(const occu_ctx *ctx, const float *X, int A, const float *Y, int Bn, long R,
-                    int splits, float *partial, cudaStream_t st);
+int launch_wgrad_tc(const occu_ctx *ctx, const float *X, int A, const void *Y, int Bn, long R,
+                    int splits, float *partial, cudaStream_t st, bool ybf = false);
 size_t tc_partial_floats(int E, int D);
 int launch_forward_layer_tc(const occu_ctx *ctx, const DevCsr &csr, int layer, const FwdLayerArgs &a,
                             float *partial, cudaStream_t st);
@@ -207,9 +213,14 @@ struct BwdLayerArgs {
   const float *de_out;                // [E][d] gradient w.r.t. e^i from layer i+1 (nullable)
   float *de_prev;                     // [E][Ke] (nullable at layer 0)
   float *dh_prev;                     // [N][K]  (nullable at layer 0)
+  bool bf = false;                    // OCCU_BF16: hbar, e, g, h and (layer > 0) h_in, e_in
+                                      // point to BF16 rows; gradients stay FP32 (R28)
 };
 int launch_backward_layer(occu_ctx *ctx, const DevCsr &csr, const BwdLayerArgs &a,
                           cudaStream_t st);
+// the backward's weight-gradient dispatcher (kernels_simt.cu), exported for occu_test_wgrad
+int launch_wgrad(occu_ctx *ctx, const float *X, int A, const void *Y, int Bn, long R, float *out,
+                 cudaStream_t st, bool ybf);
 int launch_head_backward(occu_ctx *ctx, const DevCsr &csr, const float *targets, int global_B,
                          cudaStream_t st);
 int launch_adam(occu_ctx *ctx, float lr, cudaStream_t st);

@@ -260,9 +260,9 @@ occu_status forward(occu_ctx *ctx, const DevCsr &csr, const float *nf, const flo
     a.hbar = w.hbar[i].as<float>(); a.p = w.p[i].as<float>(); a.q = w.q[i].as<float>();
     a.e_out = (!last || save_all) ? w.e[i].as<float>() : nullptr;
     a.g = w.g.as<float>();
-    if (save_all && tc && !bf && ctx->path == 0) {    // the backward reads the gates (no recompute)
+    if (save_all && tc && ctx->path == 0) {    // the backward reads the gates (no recompute)
       if (w.gs.size() < size_t(c.L)) w.gs.resize(c.L);
-      CK(w.gs[i].ensure(size_t(csr.E) * c.d * 4), "alloc saved gates");
+      CK(w.gs[i].ensure(size_t(csr.E) * c.d * (bf ? 2 : 4)), "alloc saved gates");
       a.g = w.gs[i].as<float>();
     }
     a.h_out = w.h[i].as<float>();
@@ -338,8 +338,6 @@ occu_status grads_impl(occu_ctx *ctx, const occu_batch *batch, const float *targ
   if (!batch || !batch->csr || !targets) return fail(ctx, OCCU_EINVAL, "batch/targets NULL");
   if (batch->global_num_graphs < batch->csr->num_graphs)
     return fail(ctx, OCCU_EINVAL, "global_num_graphs < local num_graphs");
-  if (ctx->cfg.prec == OCCU_BF16)
-    return fail(ctx, OCCU_EINVAL, "OCCU_BF16: training is not in this build (inference only)");
   ctx->launches = 0;
   if ((st = resolve_csr(ctx, batch->csr, csr)) != OCCU_OK) return st;
   if ((st = stage_inputs(ctx, csr, batch->node_feat, batch->edge_feat, targets, stg)) != OCCU_OK)
@@ -378,6 +376,7 @@ occu_status grads_impl(occu_ctx *ctx, const occu_batch *batch, const float *targ
     a.de_out = i < c.L - 1 ? w.deB.as<float>() : nullptr;
     a.de_prev = i > 0 ? w.deB.as<float>() : nullptr;     // read-before-write ordering, see DESIGN
     a.dh_prev = i > 0 ? w.dh.as<float>() : nullptr;
+    a.bf = c.prec == OCCU_BF16;     // h̄, e', g, h (and h_in, e_in for i > 0) stored as BF16
     LK(launch_backward_layer(ctx, csr, a, s), "backward layer");
   }
   // loss rides along the gradient buffer (slot `total`) so one allreduce sums both
@@ -618,6 +617,16 @@ occu_status occu_get_grads(const occu_ctx *cctx, float *host_flat, size_t n) {
   CK(cudaSetDevice(ctx->device), "cudaSetDevice");
   CK(cudaMemcpyAsync(host_flat, ctx->grads.ptr, n * 4, cudaMemcpyDeviceToHost, ctx->stream), "D2H");
   CK(cudaStreamSynchronize(ctx->stream), "sync");
+  return OCCU_OK;
+}
+
+occu_status occu_test_wgrad(occu_ctx *ctx, const float *X, int32_t A, const void *Y, int32_t Bn,
+                            int64_t R, int32_t y_bf16, float *out) {
+  if (!ctx || !X || !Y || !out) return fail(ctx, OCCU_EINVAL, "NULL argument");
+  if (A < 1 || Bn < 1 || R < 0 || A > 128 || Bn > 128) return fail(ctx, OCCU_EINVAL, "bad shape");
+  CK(cudaSetDevice(ctx->device), "cudaSetDevice");
+  ctx->launches = 0;
+  LK(launch_wgrad(ctx, X, A, Y, Bn, long(R), out, ctx->stream, y_bf16 != 0), "wgrad");
   return OCCU_OK;
 }
 

@@ -107,15 +107,17 @@ __device__ __forceinline__ void mma_tf32_ss(uint32_t d_tmem, uint64_t a_desc, ui
       "tcgen05.mma.cta_group::1.kind::tf32 [%0], %1, %2, %3, p;\n\t}" ::"r"(d_tmem),
       "l"(a_desc), "l"(b_desc), "r"(idsc), "r"(accumulate));
 }
-// MN-major operand, 128-byte swizzle: 32 fp32 (128 B) along M/N per row, 8 K-rows per
-// 1024-byte atom (SBO), next 32-element M/N block LBO bytes away.
-__device__ __forceinline__ uint64_t sdesc_sw128_mn(uint32_t smem_addr, uint32_t lbo_bytes) {
+// MN-major tf32 operand: the only MN-major smem layout tcgen05 accepts for 32-bit types is
+// SWIZZLE_128B_BASE32B (descriptor layout type 1): 128-byte rows of 32 fp32 along M/N, the
+// four 32-byte chunks of row k permuted by the TMA SWIZZLE_128B_ATOM_32B pattern; K-row groups
+// SBO = 512 B apart, next 32-element M/N block LBO bytes away.
+__device__ __forceinline__ uint64_t sdesc_sw128b32_mn(uint32_t smem_addr, uint32_t lbo_bytes) {
   uint64_t d = 0;
   d |= uint64_t((smem_addr >> 4) & 0x3FFF);
   d |= uint64_t((lbo_bytes >> 4) & 0x3FFF) << 16;
-  d |= uint64_t(1024 >> 4) << 32;
+  d |= uint64_t(512 >> 4) << 32;
   d |= uint64_t(1) << 46;
-  d |= uint64_t(2) << 61;
+  d |= uint64_t(1) << 61;
   return d;
 }
 

@@ -103,6 +103,7 @@ def lib():
             "occu_set_keep_intermediates": ([VP, C.c_int], I32),
             "occu_get_tensor": ([VP, I32, I32, VP, SZ], I32),
             "occu_last_launch_count": ([VP], C.c_int64),
+            "occu_test_wgrad": ([VP, VP, I32, VP, I32, C.c_int64, I32, VP], I32),
             "occu_last_error": ([VP], C.c_char_p),
             "occu_set_profiling": ([VP, C.c_int], I32),
             "occu_set_kernel_path": ([VP, C.c_int], I32),
@@ -354,6 +355,18 @@ class Model:
     def get_tensor(self, which: int, layer: int, shape) -> np.ndarray:
         out = np.empty(shape, np.float32)
         _check(lib().occu_get_tensor(self._ctx, which, layer, out.ctypes.data, out.nbytes), self._ctx)
+        return out
+
+    def test_wgrad(self, X, Y, out, y_bf16=False):
+        """Test hook: out[A][Bn] = Xᵀ Y through the backward's weight-gradient kernels
+        (torch CUDA tensors: X fp32 [R][A], Y fp32 or bf16 [R][Bn], out fp32 [A][Bn])."""
+        R, A = X.shape
+        Bn = Y.shape[1]
+        for t in (X, Y, out):
+            if not (t.is_cuda and t.is_contiguous()):
+                raise ValueError("contiguous CUDA tensors expected")
+        _check(lib().occu_test_wgrad(self._ctx, X.data_ptr(), A, Y.data_ptr(), Bn, R,
+                                     int(y_bf16), out.data_ptr()), self._ctx)
         return out
 
     def last_launch_count(self) -> int:

@@ -354,3 +354,6 @@ def test_cfg3_full_size_training_properties():
         m.compute_grads(hc, hn, he, hy, global_num_graphs=512)
         g_sum += m.get_grads().astype(np.float64)
     assert rel(g_full, g_sum) <= 1e-5, rel(g_full, g_sum)
+    # every parameter tensor receives a gradient (the identity above holds trivially for 0)
+    for k, v in weights.unflatten(wcfg(c), g_full).items():
+        assert np.linalg.norm(v) > 0, k
