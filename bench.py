@@ -213,14 +213,14 @@ def cpu_baseline_sample(seconds=12.0):
     params = oracle.unflatten(ocf, weights.init_flat(wc, 42).astype(np.float64))
     full = configs.cfg2(256)
     done, t0 = 0, time.perf_counter()
-    while time.perf_counter() - t0 < seconds and done < 256:
-        s = full.subset([done, done + 1])
+    while time.perf_counter() - t0 < seconds:
+        s = full.subset([done % 256, (done + 1) % 256])
         oracle.predict(params, ocf, s.graphs, s.node_feat, s.edge_feat)
         done += 2
     dt = time.perf_counter() - t0
     return {"value": done / dt, "unit": "graphs/s", "cores": cpu_cores_used(), "kind": "oracle",
-            "sample": f"{done} CFG2 ResNet-50 graphs (L=3, d=128), float64 NumPy oracle forward, "
-                      f"{dt:.1f} s"}
+            "sample": f"{done} CFG2 ResNet-50 graphs (L=3, d=128; the 256-graph batch cycled, "
+                      f"2 graphs per oracle call), float64 NumPy oracle forward, {dt:.1f} s"}
 
 
 def main():
@@ -447,6 +447,27 @@ def main():
                  "kernel_ms_per_step": {k: v[0] / args.steps for k, v in tprof.items()},
                  "includes": "forward with saves, MSE, backward, "
                              + ("NCCL allreduce, " if world > 1 else "") + "Adam"}
+        if not args.no_bf16 and args.path == 0:
+            # OCCU_BF16 training step (R28): BF16 saves, FP32 gradients and Adam
+            mb = occu.Model(occu.config(L=3, F_n=80, F_e=4, d=128, prec=occu.BF16), device=local,
+                            stream=stream.cuda_stream)
+            mb.init_weights(42)
+            if pg and world > 1:
+                uid = [occu.Model.nccl_unique_id() if rank == 0 else None]
+                pg.broadcast_object_list(uid, src=0)
+                mb.dist_init(rank, world, uid[0])
+            stepb = lambda: mb.train_step(csr, nf, ef, yt, 1e-4, global_num_graphs=gB, want_loss=False)
+            timed(stepb, args.warmup, mdl=mb)
+            bar()
+            bt, bl = timed(stepb, args.steps, profile=True, mdl=mb)
+            bar()
+            bprof = mb.profile()
+            bms = max_over_ranks(float(np.sum(bt)) / args.steps)
+            train["bf16"] = {"value": gB / (bms * 1e-3), "unit": "graphs/s", "ms_per_step": bms,
+                             "dtype": "bf16", "gpu_launches": bl,
+                             "loss_after": mb.train_step(csr, nf, ef, yt, 1e-4, global_num_graphs=gB),
+                             "kernel_ms_per_step": {k: v[0] / args.steps for k, v in bprof.items()}}
+            del mb
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu:
