@@ -30,6 +30,11 @@ constexpr int NT = 256;
 __device__ __forceinline__ float lrelu(float x, float s) { return x > 0.f ? x : s * x; }
 __device__ __forceinline__ float lrelu_grad_from_out(float y, float s) { return y > 0.f ? 1.f : s; }
 __device__ __forceinline__ float sigmoidf_(float x) { return 1.f / (1.f + expf(-x)); }
+__device__ __forceinline__ float ex2f_fast(float x) {     // MUFU.EX2 (~2 ulp); ex2(-inf) = 0
+  float r;
+  asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(r) : "f"(x));
+  return r;
+}
 // Element i of an FP32 or (BF = true) BF16 stored activation (OCCU_BF16 training, R28).
 template <bool BF> __device__ __forceinline__ float ld_act(const void *base, long i) {
   if constexpr (BF)
@@ -617,11 +622,16 @@ __global__ void __launch_bounds__(NT, (BF ? G <= 8 : G == 4) ? 4 : 3) gather_seg
 // A warp takes 32 consecutive in-CSR edges, four at a time with all row loads of the
 // four in flight; lane = D/32 channels; the dot is a fixed-order butterfly.
 // ---------------------------------------------------------------------------
-template <int D, bool BF>
+// MSGB (reading B, NEXT-1): g holds the per-channel in-edge softmax weights w; the segmented
+// softmax backward dv_k = w_k ⊙ (dg_k - Σ_{k'∈seg(t)} w_k' ⊙ dg_k') with dg_k = dA_t ⊙ h̄[s_k]
+// has Σ_{k'} w_k' ⊙ dg_k' = dA_t ⊙ A_t (A_t = Σ_k' w_k' ⊙ h̄[s_k'], the un-divided segment sum,
+// recovered from h_t = LReLU(A_t / deg_t)), so dv_k = w_k ⊙ dA_t ⊙ (h̄[s_k] - A_t).
+template <int D, bool BF, bool MSGB = false>
 __global__ void __launch_bounds__(NT) gate_bwd_stream_kernel(
     const void *__restrict__ g, const float *__restrict__ dA, const void *__restrict__ hbar,
     const int32_t *__restrict__ in_src, const int32_t *__restrict__ in_dst, int E,
-    float *__restrict__ MG, float *__restrict__ DV) {
+    float *__restrict__ MG, float *__restrict__ DV, const float *__restrict__ h = nullptr,
+    const int32_t *__restrict__ in_ptr = nullptr, int mean = 0, float slope = 0.01f) {
   constexpr int V = D / 32;
   constexpr int G = 4;
   const int lane = threadIdx.x & 31;
@@ -632,13 +642,23 @@ __global__ void __launch_bounds__(NT) gate_bwd_stream_kernel(
     const int t_l = lane < cnt ? __ldg(in_dst + k0 + lane) : 0;
     for (int j = 0; j < cnt; j += G) {
       RawRow<V, BF> gr[G], hr[G];
-      RawRow<V, false> dr[G];
+      RawRow<V, false> dr[G], ar[MSGB ? G : 1];
+      float dsc[MSGB ? G : 1];
 #pragma unroll
       for (int u = 0; u < G; ++u) {
         const int kk = min(j + u, cnt - 1);
+        const int tk = __shfl_sync(0xffffffffu, t_l, kk);
         gr[u].load(g, k0 + kk, D, lane);
-        dr[u].load(dA, __shfl_sync(0xffffffffu, t_l, kk), D, lane);
+        dr[u].load(dA, tk, D, lane);
         hr[u].load(hbar, __shfl_sync(0xffffffffu, s_l, kk), D, lane);
+        if constexpr (MSGB) {
+          ar[u].load(h, tk, D, lane);
+          dsc[u] = 1.f;
+          if (mean) {
+            const int deg = __ldg(in_ptr + tk + 1) - __ldg(in_ptr + tk);
+            dsc[u] = float(deg > 0 ? deg : 1);
+          }
+        }
       }
 #pragma unroll
       for (int u = 0; u < G; ++u) {
@@ -647,6 +667,19 @@ __global__ void __launch_bounds__(NT) gate_bwd_stream_kernel(
         gr[u].get(gv);
         dr[u].get(dv);
         hr[u].get(hv);
+        if constexpr (MSGB) {
+          float av[V], mg[V], dvv[V];
+          ar[u].get(av);
+#pragma unroll
+          for (int c = 0; c < V; ++c) {
+            const float At = (av[c] > 0.f ? av[c] : av[c] / slope) * dsc[u];   // LReLU⁻¹, × deg
+            mg[c] = dv[c] * gv[c];
+            dvv[c] = mg[c] * (hv[c] - At);
+          }
+          store_row<V>(MG + (k0 + j + u) * D + lane * V, mg);
+          store_row<V>(DV + (k0 + j + u) * D + lane * V, dvv);
+          continue;
+        }
         double dot = 0.0;
 #pragma unroll
         for (int c = 0; c < V; ++c) {
@@ -665,6 +698,132 @@ __global__ void __launch_bounds__(NT) gate_bwd_stream_kernel(
         store_row<V>(MG + (k0 + j + u) * D + lane * V, mg);
         store_row<V>(DV + (k0 + j + u) * D + lane * V, dvv);
       }
+    }
+  }
+}
+
+// ---------------------------------------------------------------------------
+// a4-a6 under reading B (NEXT-1; P149 with the softmax taken over the in-edges
+// of the destination, per channel): with logits v_k = W_m e'_k (tensor-core plain GEMM),
+//   w_kc = exp(v_kc - M_tc) / Σ_{k'∈seg(t)} exp(v_k'c - M_tc),   A_tc = Σ_{k∈seg(t)} w_kc h̄[s_k]c
+// h_t = LReLU(A_t) (÷ deg for MEAN; an empty segment gives 0).  One pass per segment with an
+// online maximum and rescaled running sums per lane-channel, edges in ascending in-CSR order
+// (fixed order, atomic-free).  Warps walk chunks of 8 destinations; G (v, h̄[s]) row pairs of
+// the chunk are in flight at a time.  W (training): a second pass over each finished segment
+// overwrites v_k with w_k (the weights the backward reads; each row is read before it is
+// written and only by its owner warp).  RP: last layer, readout chunk partials as v2.
+// ---------------------------------------------------------------------------
+template <int D, int G, bool RP, bool W>
+__global__ void __launch_bounds__(NT) gather_segsoftmax_kernel(
+    float *__restrict__ v, const float *__restrict__ hbar, const int32_t *__restrict__ in_ptr,
+    const int32_t *__restrict__ in_src, int N, int mean, float slope, float *__restrict__ h_out,
+    const int32_t *__restrict__ node_graph, float *__restrict__ rpart) {
+  constexpr int V = D / 32;
+  constexpr int NPW = 8;
+  constexpr float L2E = 1.4426950408889634f;
+  const int lane = threadIdx.x & 31;
+  const long nw = (long(gridDim.x) * NT) / 32;
+  pdl_trigger();
+  pdl_wait();
+  for (long t0 = (blockIdx.x * long(NT) + threadIdx.x) / 32 * NPW; t0 < N; t0 += nw * NPW) {
+    const int nn = int(min(long(NPW), N - t0));
+    const int ptr_l = lane <= nn ? __ldg(in_ptr + t0 + lane) : 0;
+    const int gr_l = (RP && lane < nn) ? __ldg(node_graph + t0 + lane) : -1;
+    const int e_beg = __shfl_sync(0xffffffffu, ptr_l, 0);
+    const int e_end = __shfl_sync(0xffffffffu, ptr_l, nn);
+    int node = 0;
+    int seg_beg = e_beg;
+    int seg_end = __shfl_sync(0xffffffffu, ptr_l, 1);
+    float m[V], sum[V], acc[V], racc[V];
+#pragma unroll
+    for (int c = 0; c < V; ++c) {
+      m[c] = -INFINITY;
+      sum[c] = acc[c] = racc[c] = 0.f;
+    }
+    auto flush = [&](int nd) {
+      const int deg = seg_end - seg_beg;
+      float o[V];
+#pragma unroll
+      for (int c = 0; c < V; ++c) {
+        float x = deg > 0 ? acc[c] / sum[c] : 0.f;
+        if (mean) x = x / float(deg > 0 ? deg : 1);
+        o[c] = lrelu(x, slope);
+      }
+      if (W && deg > 0) {                   // weights of the finished segment, in place
+        float inv[V];
+#pragma unroll
+        for (int c = 0; c < V; ++c) inv[c] = 1.f / sum[c];
+        for (int k = seg_beg; k < seg_end; ++k) {
+          float x[V];
+          load_row<V, false>(v, long(k), D, lane, x);
+#pragma unroll
+          for (int c = 0; c < V; ++c) x[c] = ex2f_fast((x[c] - m[c]) * L2E) * inv[c];
+          store_row<V>(v + long(k) * D + lane * V, x);
+        }
+      }
+#pragma unroll
+      for (int c = 0; c < V; ++c) {
+        m[c] = -INFINITY;
+        sum[c] = acc[c] = 0.f;
+      }
+      if (!RP || h_out) store_row_t<V, false>(h_out, t0 + nd, D, lane, o);
+      if (RP) {
+        const int gc = __shfl_sync(0xffffffffu, gr_l, nd);
+        const int gn = __shfl_sync(0xffffffffu, gr_l, (nd + 1) & 31);
+#pragma unroll
+        for (int c = 0; c < V; ++c) racc[c] += o[c];
+        if (nd + 1 >= nn || gn != gc) {
+          store_row<V>(rpart + (t0 + nd) * D + lane * V, racc);
+#pragma unroll
+          for (int c = 0; c < V; ++c) racc[c] = 0.f;
+        }
+      }
+    };
+    for (int base = e_beg; base < e_end; base += 32) {
+      const int cnt = min(32, e_end - base);
+      const int s_l = lane < cnt ? __ldg(in_src + base + lane) : 0;
+      for (int j = 0; j < cnt; j += G) {
+        RawRow<V, false> vr[G], hr[G];
+#pragma unroll
+        for (int u = 0; u < G; ++u) {
+          const int kk = min(j + u, cnt - 1);
+          vr[u].load(v, long(base + kk), D, lane);
+          hr[u].load(hbar, long(__shfl_sync(0xffffffffu, s_l, kk)), D, lane);
+        }
+#pragma unroll
+        for (int u = 0; u < G; ++u) {
+          if (j + u < cnt) {
+            const int k = base + j + u;
+            while (k >= seg_end) {
+              flush(node);
+              ++node;
+              seg_beg = seg_end;
+              seg_end = __shfl_sync(0xffffffffu, ptr_l, node + 1);
+            }
+            float xv[V], hv[V];
+            vr[u].get(xv);
+            hr[u].get(hv);
+#pragma unroll
+            for (int c = 0; c < V; ++c) {
+              if (xv[c] > m[c]) {            // new maximum: rescale the running sums
+                const float sc = ex2f_fast((m[c] - xv[c]) * L2E);
+                sum[c] = fmaf(sum[c], sc, 1.f);
+                acc[c] = fmaf(acc[c], sc, hv[c]);
+                m[c] = xv[c];
+              } else {
+                const float e = ex2f_fast((xv[c] - m[c]) * L2E);
+                sum[c] += e;
+                acc[c] = fmaf(e, hv[c], acc[c]);
+              }
+            }
+          }
+        }
+      }
+    }
+    for (; node < nn; ++node) {
+      flush(node);
+      seg_beg = seg_end;
+      seg_end = __shfl_sync(0xffffffffu, ptr_l, min(node + 2, nn));
     }
   }
 }
@@ -1387,6 +1546,36 @@ static int gather_bf16_impl(const occu_ctx *ctx, const DevCsr &csr, const void *
   return 1;
 }
 
+template <int D>
+static int segsoftmax_impl(const occu_ctx *ctx, const DevCsr &csr, float *v, const float *hbar,
+                           float *h_out, float *rpart, bool write_w, cudaStream_t st) {
+  if (csr.N <= 0) return 0;
+  const int mean = ctx->cfg.aggr == OCCU_AGGR_MEAN;
+  const int grid = grid_for(long(csr.N) * 4, NT, 8 * ctx->num_sms);
+  OCCU_PROF_BEGIN(ctx, "gather_segsoftmax", st);
+#define OCCU_GS_ARGS v, hbar, csr.in_ptr, csr.in_src, csr.N, mean, ctx->cfg.slope, h_out, csr.node_graph, rpart
+  if (write_w) {
+    if (rpart) launch_pdl(ctx->pdl & 2, gather_segsoftmax_kernel<D, 4, true, true>, grid, NT, 0, st, OCCU_GS_ARGS);
+    else launch_pdl(ctx->pdl & 2, gather_segsoftmax_kernel<D, 4, false, true>, grid, NT, 0, st, OCCU_GS_ARGS);
+  } else {
+    if (rpart) launch_pdl(ctx->pdl & 2, gather_segsoftmax_kernel<D, 4, true, false>, grid, NT, 0, st, OCCU_GS_ARGS);
+    else launch_pdl(ctx->pdl & 2, gather_segsoftmax_kernel<D, 4, false, false>, grid, NT, 0, st, OCCU_GS_ARGS);
+  }
+#undef OCCU_GS_ARGS
+  OCCU_PROF_END(ctx);
+  LAUNCH_CHECK();
+  return 1;
+}
+
+int launch_gather_segsoftmax(const occu_ctx *ctx, const DevCsr &csr, float *v, const float *hbar,
+                             float *h_out, float *rpart, bool write_w, cudaStream_t st) {
+  switch (ctx->cfg.d) {
+    case 64: return segsoftmax_impl<64>(ctx, csr, v, hbar, h_out, rpart, write_w, st);
+    case 128: return segsoftmax_impl<128>(ctx, csr, v, hbar, h_out, rpart, write_w, st);
+    default: return -int(cudaErrorInvalidValue);
+  }
+}
+
 int launch_gather_segsum_bf16(const occu_ctx *ctx, const DevCsr &csr, const void *g,
                               const void *hbar, void *h_out, float *rpart, cudaStream_t st) {
   switch (ctx->cfg.d) {
@@ -1551,12 +1740,20 @@ static int backward_layer_impl(occu_ctx *ctx, const DevCsr &csr, const BwdLayerA
   const bool tc = ctx->path != 1 && tc_supported(cf);
   const bool bf = a.bf;                     // OCCU_BF16: stored activations are BF16 (R28)
   const bool in_bf = bf && i > 0;           // h_in, e_in of layer 1 are the FP32 inputs
-  if (bf && !(tc && a.g)) return -int(cudaErrorInvalidValue);
+  if ((bf || cf.msg == OCCU_MSG_NEIGHBOR_SOFTMAX) && !(tc && a.g)) return -int(cudaErrorInvalidValue);
   int r;
   if (tc && csr.E > 0) {
     // a10: softmax / message backward (streaming with the saved gates, else g recomputed on
     // tensor cores), W_mᵀ dv, z recompute + σ', W_eᵀ dz on tensor cores
-    if (a.g) {
+    if (a.g && cf.msg == OCCU_MSG_NEIGHBOR_SOFTMAX) {
+      OCCU_PROF_BEGIN(ctx, "gate_bwd", st);
+      gate_bwd_stream_kernel<D, false, true><<<grid_for((long(csr.E) + 31) / 32, NT / 32, 8 * sms), NT, 0, st>>>(
+          a.g, a.dh, a.hbar, csr.in_src, csr.in_dst, csr.E, w.MG.as<float>(), w.DV.as<float>(),
+          a.h, csr.in_ptr, cf.aggr == OCCU_AGGR_MEAN, cf.slope);
+      OCCU_PROF_END(ctx);
+      LAUNCH_CHECK();
+      ++n;
+    } else if (a.g) {
       OCCU_PROF_BEGIN(ctx, "gate_bwd", st);
       if (bf)
         gate_bwd_stream_kernel<D, true><<<grid_for((long(csr.E) + 31) / 32, NT / 32, 8 * sms), NT, 0, st>>>(

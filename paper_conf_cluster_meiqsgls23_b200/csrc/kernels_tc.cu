@@ -181,12 +181,16 @@ __device__ __forceinline__ Smem carve(uint8_t *raw, int D, int K) {
   return s;
 }
 
-// e such that max|x|·2^e lies in [2^14, 2^15); 0 for an all-zero row.
+// e such that max|x|·2^e lies in [2^14, 2^15); 0 for an all-zero row.  Capped at 100 so that
+// 2^e stays finite and the epilogue's 2^-(e_row + f) (f <= ~30 for the weights) stays a
+// representable power of two: a row whose largest entry is below 2^-86 keeps less than 22
+// significant bits in fp16x2, an absolute error below 2^-108 (without the cap 2^e overflowed
+// to inf and such rows came out NaN — seen on tiny gradient rows under reading B + MEAN).
 __device__ __forceinline__ int scale_exp(float mx) {
   if (!(mx > 0.f) || !isfinite(mx)) return 0;
   int E;
   frexpf(mx, &E);
-  return 15 - E;
+  return min(15 - E, 100);
 }
 
 // x (already scaled) -> packed fp16 pair hi and lo for elements (v0, v1).
@@ -1798,7 +1802,7 @@ static int tc_forward_layer_impl(const occu_ctx *ctx, const DevCsr &csr, int lay
   ra.rev = ctx->l2_order;
   if ((r = launch_rowgemm<D, EPI_NODE>(ctx, ra, "node_tc", st)) < 0) return r;
   n += r;
-  const bool fused_eg = ctx->path == 0 && ctx->fuse_edge_gate &&
+  const bool fused_eg = ctx->path == 0 && ctx->fuse_edge_gate && ctx->cfg.msg == OCCU_MSG_CHANNEL_SOFTMAX &&
                         (a.Ke <= 16 || (a.Ke % 64 == 0 && a.Ke <= 128));
   if (csr.E > 0 && fused_eg) {
     // a3 + a4 fused: e' and g in one kernel (e' is not re-read)
@@ -1837,6 +1841,11 @@ static int tc_forward_layer_impl(const occu_ctx *ctx, const DevCsr &csr, int lay
       rg.mean = ctx->cfg.aggr == OCCU_AGGR_MEAN; rg.part = partial;
       if ((r = launch_rowgemm<D, EPI_GATEAGG>(ctx, rg, "gate_agg_tc", st)) < 0) return r;
       n += r;
+    } else if (ctx->cfg.msg == OCCU_MSG_NEIGHBOR_SOFTMAX) {
+      // a4 under reading B: logits v = W_m e' -> g (the softmax runs in the aggregation)
+      if ((r = launch_plain_tc(ctx, a.e_out, D, csr.E, 2, layer, nullptr, a.g, "gate_tc", st)) < 0)
+        return r;
+      n += r;
     } else {
       // a4: channel-softmax gate -> g
       RowGemmArgs rg{};
@@ -1858,6 +1867,11 @@ static int tc_forward_layer_impl(const occu_ctx *ctx, const DevCsr &csr, int lay
       TC_CHECK();
       ++n;
     }
+  } else if (ctx->cfg.msg == OCCU_MSG_NEIGHBOR_SOFTMAX) {
+    // a5 + a6 under reading B: segmented per-channel softmax + message + sum
+    if ((r = launch_gather_segsoftmax(ctx, csr, a.g, a.hbar, a.h_out, a.rpart, a.save_w, st)) < 0)
+      return r;
+    n += r;
   } else {
     // a5 + a6: gather + segmented sum (CUDA cores, warp per 8 destinations)
     if ((r = launch_gather_segsum(ctx, csr, a.g, a.hbar, a.h_out, a.rpart, st)) < 0) return r;

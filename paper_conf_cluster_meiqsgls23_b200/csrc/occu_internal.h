@@ -159,6 +159,7 @@ struct FwdLayerArgs {
   // the last layer's aggregation emits readout chunk partials into rpart (h_out may
   // then be null).  See gather_segsum_kernel / readout_head_kernel.
   const int32_t *e_eid; float *e0_out; float *rpart;
+  bool save_w = false;                 // reading B, training: g receives the softmax weights
 };
 int launch_forward_layer(const occu_ctx *ctx, const DevCsr &csr, const FwdLayerArgs &a,
                          cudaStream_t st);
@@ -190,6 +191,11 @@ int launch_forward_layer_tc(const occu_ctx *ctx, const DevCsr &csr, int layer, c
                             float *partial, cudaStream_t st);
 int launch_gather_segsum(const occu_ctx *ctx, const DevCsr &csr, const float *g,
                          const float *hbar, float *h_out, float *rpart, cudaStream_t st);
+// Reading B (OCCU_MSG_NEIGHBOR_SOFTMAX, NEXT-1): v holds the logits W_m e'; the per-channel
+// softmax over each destination's in-edges, the message product and the segmented sum in one
+// pass; write_w (training) overwrites v with the softmax weights for the backward.
+int launch_gather_segsoftmax(const occu_ctx *ctx, const DevCsr &csr, float *v, const float *hbar,
+                             float *h_out, float *rpart, bool write_w, cudaStream_t st);
 // OCCU_BF16: g, h̄, h stored as BF16 (FP32 arithmetic); rpart stays FP32.
 int launch_gather_segsum_bf16(const occu_ctx *ctx, const DevCsr &csr, const void *g,
                               const void *hbar, void *h_out, float *rpart, cudaStream_t st);

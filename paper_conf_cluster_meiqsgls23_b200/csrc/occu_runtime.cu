@@ -153,8 +153,10 @@ occu_status validate_cfg(const occu_config *c) {
   if (c->d_h < 1 || c->d_h > 1024) return fail(nullptr, OCCU_EINVAL, "d_h must be in [1, 1024]");
   if (c->aggr != OCCU_AGGR_SUM && c->aggr != OCCU_AGGR_MEAN)
     return fail(nullptr, OCCU_EINVAL, "aggr must be SUM or MEAN");
-  if (c->msg != OCCU_MSG_CHANNEL_SOFTMAX)
-    return fail(nullptr, OCCU_EINVAL, "msg: only OCCU_MSG_CHANNEL_SOFTMAX (reading A) in this build");
+  if (c->msg != OCCU_MSG_CHANNEL_SOFTMAX && c->msg != OCCU_MSG_NEIGHBOR_SOFTMAX)
+    return fail(nullptr, OCCU_EINVAL, "msg must be CHANNEL_SOFTMAX (reading A) or NEIGHBOR_SOFTMAX (reading B)");
+  if (c->msg == OCCU_MSG_NEIGHBOR_SOFTMAX && (c->prec != OCCU_FP32 || c->F_n > 128))
+    return fail(nullptr, OCCU_EINVAL, "reading B (NEIGHBOR_SOFTMAX) runs in OCCU_FP32 on the tensor-core path (F_n <= 128)");
   if (c->prec != OCCU_FP32 && c->prec != OCCU_BF16)
     return fail(nullptr, OCCU_EINVAL, "prec must be OCCU_FP32 or OCCU_BF16");
   if (c->prec == OCCU_BF16 && !(c->F_n <= 128 && (c->F_e <= 16 || c->F_e % 64 == 0)))
@@ -266,6 +268,7 @@ occu_status forward(occu_ctx *ctx, const DevCsr &csr, const float *nf, const flo
       a.g = w.gs[i].as<float>();
     }
     a.h_out = w.h[i].as<float>();
+    a.save_w = save_all && c.msg == OCCU_MSG_NEIGHBOR_SOFTMAX;   // reading B: weights for the backward
     if (tc) {
       a.e_out = w.e[i].as<float>();            // the gate kernel re-reads e'
       if (last && fuse_ro) {
@@ -705,6 +708,8 @@ occu_status occu_set_kernel_path(occu_ctx *ctx, int path) {
     return fail(ctx, OCCU_EINVAL, "path must be 0 (tensor cores), 1 (SIMT) or 2 (tensor cores, fused aggregation)");
   if (ctx->cfg.prec == OCCU_BF16 && path != 0)
     return fail(ctx, OCCU_EINVAL, "OCCU_BF16 runs on kernel path 0 only");
+  if (ctx->cfg.msg == OCCU_MSG_NEIGHBOR_SOFTMAX && path != 0)
+    return fail(ctx, OCCU_EINVAL, "reading B (NEIGHBOR_SOFTMAX) runs on kernel path 0 only");
   ctx->path = path;
   return OCCU_OK;
 }
