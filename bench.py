@@ -146,6 +146,33 @@ def algorithmic_bytes(N, E, B, d=128, F_n=80, F_e=4, L=3, rrows=None, sa=4):
     return out
 
 
+def train_algorithmic_bytes(N, E, B, d=128, F_n=80, F_e=4, L=3, rrows=0, sa=4):
+    """Per-step algorithmic bytes of the training step's kernels: every
+    operand read once and every result written once; sa = stored-activation bytes (h̄, e', g,
+    h: 4 FP32, 2 BF16), gradients and the backward's scratch (dA, MG, DV, DZ, de, dP) FP32.
+    The split-K partials of the weight gradients are an artefact of the kernel design and
+    count 0."""
+    s = 4
+    fwd = algorithmic_bytes(N, E, B, d, F_n, F_e, L, rrows=rrows, sa=sa)
+    out = {k: fwd[k] for k in ("node_tc", "edge_small", "edge_tc", "gate_tc", "readout_head")}
+    # forward with saves: the last layer also stores e' (edge kernels) and h (gather)
+    out["gather_segsum"] = fwd["gather_segsum"] + sa * N * d
+    out["broadcast_dh"] = sa * N * d + s * N * d + 4 * N
+    Ed, Nd = E * d, N * d
+    out["gate_bwd"] = L * (sa * Ed + s * Nd + sa * Nd + 2 * s * Ed + 8 * E)
+    out["de_tc"] = L * (2 * s * Ed) + (L - 1) * s * Ed
+    out["edge_bwd_tc"] = (L - 1) * (2 * sa * Ed + s * Ed + 8 * N + 8 * E + s * Ed + 4 * E)
+    out["edge_bwd_e"] = s * E * F_e + sa * Ed + s * Ed + 8 * N + 8 * E + s * Ed + 4 * E
+    out["de_prev_tc"] = (L - 1) * 2 * s * Ed
+    out["node_bwd"] = L * (s * Ed + 8 * E + sa * Nd + s * Nd + 8 * N + 8 * N + 4 * E)
+    out["wgrad_tc"] = (L * (s * Ed + sa * Ed) + (L - 1) * (s * Ed + sa * Ed)
+                       + (s * Nd + s * N * F_n) + (L - 1) * (s * Nd + sa * Nd))
+    out["wgrad_skinny"] = s * Ed + s * E * F_e
+    out["dh_prev_tc"] = (L - 1) * (2 * s * Nd + sa * Nd)
+    out["split_reduce"] = 0
+    return out
+
+
 def load_traffic(name="traffic.json"):
     """Per-launch DRAM bytes (ncu dram__bytes_read+write) committed under profiles/."""
     try:
@@ -401,6 +428,31 @@ def main():
                 "kernel_ms_per_step": {k: v["ms_per_step"] for k, v in kb.items()}, "kernels": kb}
         del mb
 
+    # ---- reading B (NEXT-1, OCCU_MSG_NEIGHBOR_SOFTMAX) inference on the same CFG2 batch
+    readingb = None
+    if not args.no_bf16 and args.path == 0:
+        mr = occu.Model(occu.config(L=3, F_n=80, F_e=4, d=128, msg=occu.MSG_NEIGHBOR_SOFTMAX),
+                        device=local, stream=stream.cuda_stream)
+        mr.init_weights(42)
+        outr = torch.empty_like(out)
+        inferr = lambda: mr.predict(csr, nf, ef, outr)
+        timed(inferr, args.warmup, mdl=mr)
+        bar()
+        tr_, lr_ = timed(inferr, args.steps, mdl=mr)
+        bar()
+        timed(inferr, args.steps, profile=True, mdl=mr)
+        bar()
+        msr = max_over_ranks(float(np.sum(tr_)) / args.steps)
+        algr = dict(alg)
+        algr["gather_segsoftmax"] = alg["gather_segsum"]       # same rows moved
+        algr["gate_tc"] = alg["gate_tc"]                        # logits instead of gates, same bytes
+        kr, roofr = kernel_table(mr.profile(), algr, {})
+        readingb = {"value": B * world / (msr * 1e-3), "unit": "graphs/s", "ms_per_step": msr,
+                    "dtype": "f32", "gpu_launches": lr_, "roofline": roofr,
+                    "kernel_ms_per_step": {k: v["ms_per_step"] for k, v in kr.items()}, "kernels": kr,
+                    "what": "ANEE reading B: per-channel softmax over each destination's in-edges"}
+        del mr
+
     # ---- e2e through the public API with host buffers (pinned), pack included
     pin_nf = torch.from_numpy(batch.node_feat).pin_memory()
     pin_ef = torch.from_numpy(batch.edge_feat).pin_memory()
@@ -442,8 +494,15 @@ def main():
         tprof = model.profile()
         tms = max_over_ranks(float(np.sum(ttimes)) / args.steps)
         loss = model.train_step(csr, nf, ef, yt, 1e-4, global_num_graphs=gB)
+        talg = train_algorithmic_bytes(N, E, B, d, rrows=rrows)
+        tk, troof = kernel_table(tprof, talg, load_traffic())
+        tot_alg = sum(v for k, v in talg.items() if k in tprof)
         train = {"value": gB / (tms * 1e-3), "unit": "graphs/s", "ms_per_step": tms,
                  "global_batch": gB, "gpu_launches": tl, "loss_after": loss,
+                 "roofline": troof,
+                 "step_algorithmic_bytes": tot_alg,
+                 "step_frac_of_hbm": tot_alg / (tms * 1e-3) / 1e9 / peaks["hbm_gbs"],
+                 "kernels": tk,
                  "kernel_ms_per_step": {k: v[0] / args.steps for k, v in tprof.items()},
                  "includes": "forward with saves, MSE, backward, "
                              + ("NCCL allreduce, " if world > 1 else "") + "Adam"}
@@ -463,8 +522,14 @@ def main():
             bar()
             bprof = mb.profile()
             bms = max_over_ranks(float(np.sum(bt)) / args.steps)
+            balg = train_algorithmic_bytes(N, E, B, d, rrows=rrows, sa=2)
+            bk, broof = kernel_table(bprof, balg, {})
+            btot = sum(v for k, v in balg.items() if k in bprof)
             train["bf16"] = {"value": gB / (bms * 1e-3), "unit": "graphs/s", "ms_per_step": bms,
-                             "dtype": "bf16", "gpu_launches": bl,
+                             "dtype": "bf16", "gpu_launches": bl, "roofline": broof,
+                             "step_algorithmic_bytes": btot,
+                             "step_frac_of_hbm": btot / (bms * 1e-3) / 1e9 / peaks["hbm_gbs"],
+                             "kernels": bk,
                              "loss_after": mb.train_step(csr, nf, ef, yt, 1e-4, global_num_graphs=gB),
                              "kernel_ms_per_step": {k: v[0] / args.steps for k, v in bprof.items()}}
             del mb
@@ -495,6 +560,7 @@ def main():
                               "ms_per_step_with_events": ms_step_prof},
             "e2e": e2e,
             "bf16": bf16,
+            "readingb": readingb,
             "train": train,
             "cpu_baseline": cpu,
         }

@@ -828,6 +828,92 @@ __global__ void __launch_bounds__(NT) gather_segsoftmax_kernel(
   }
 }
 
+// ---------------------------------------------------------------------------
+// a10, layer-1 edge backward (F_e = Ke <= KM small; the edge transform was a CUDA-core step):
+//   z = W_e e0_k (recomputed from the saved permuted features), y = α z,
+//   dy = de ⊙ e' ⊙ σ(-y), dα = <dy, z> (float64), DZ = α dy.
+// A warp takes 32 consecutive in-CSR edges: lane j loads edge j's α and Ke features (all in
+// flight), then the warp walks the edges four at a time with the e' / de rows of the four in
+// flight; lane = D/32 channels (coalesced rows), W_e's columns for the lane's channels live in
+// registers; the dot is a fixed-order butterfly.  BF: e' rows are BF16 (OCCU_BF16 training).
+// ---------------------------------------------------------------------------
+template <int D, int KM, bool BF>
+__global__ void __launch_bounds__(NT) edge_bwd_small_kernel(
+    const float *__restrict__ e0, int Ke, const void *__restrict__ e, const float *__restrict__ de,
+    const float *__restrict__ W_e, const float *__restrict__ p, const float *__restrict__ q,
+    const int32_t *__restrict__ in_src, const int32_t *__restrict__ in_dst, int E,
+    float *__restrict__ DZ, float *__restrict__ dalpha) {
+  constexpr int V = D / 32;
+  constexpr int G = 4;
+  constexpr float L2E = 1.4426950408889634f;
+  const int lane = threadIdx.x & 31;
+  float w[KM][V];
+#pragma unroll
+  for (int j = 0; j < KM; ++j)
+#pragma unroll
+    for (int c = 0; c < V; ++c) w[j][c] = j < Ke ? __ldg(W_e + long(lane * V + c) * Ke + j) : 0.f;
+  const long nwarps = long(gridDim.x) * (NT / 32);
+  for (long k0 = (blockIdx.x * long(NT / 32) + threadIdx.x / 32) * 32; k0 < E; k0 += nwarps * 32) {
+    const int cnt = int(min(32L, E - k0));
+    float al = 0.f, ev[KM];
+#pragma unroll
+    for (int j = 0; j < KM; ++j) ev[j] = 0.f;
+    if (lane < cnt) {
+      const long k = k0 + lane;
+      al = __ldg(p + __ldg(in_src + k)) + __ldg(q + __ldg(in_dst + k));
+      if (KM == 4 && Ke == 4) {
+        const float4 x = __ldg(reinterpret_cast<const float4 *>(e0 + k * 4));
+        ev[0] = x.x; ev[1 % KM] = x.y; ev[2 % KM] = x.z; ev[3 % KM] = x.w;
+      } else {
+#pragma unroll
+        for (int j = 0; j < KM; ++j) ev[j] = j < Ke ? __ldg(e0 + k * Ke + j) : 0.f;
+      }
+    }
+    float dal_mine = 0.f;
+    for (int jb = 0; jb < cnt; jb += G) {
+      RawRow<V, BF> er[G];
+      RawRow<V, false> dr[G];
+#pragma unroll
+      for (int u = 0; u < G; ++u) {
+        const int kk = min(jb + u, cnt - 1);
+        er[u].load(e, k0 + kk, D, lane);
+        dr[u].load(de, k0 + kk, D, lane);
+      }
+#pragma unroll
+      for (int u = 0; u < G; ++u) {
+        if (jb + u >= cnt) break;                       // warp-uniform
+        const int kk = jb + u;
+        const float a = __shfl_sync(0xffffffffu, al, kk);
+        float z[V];
+#pragma unroll
+        for (int c = 0; c < V; ++c) z[c] = 0.f;
+#pragma unroll
+        for (int j = 0; j < KM; ++j) {
+          const float x = __shfl_sync(0xffffffffu, ev[j], kk);
+#pragma unroll
+          for (int c = 0; c < V; ++c) z[c] = fmaf(w[j][c], x, z[c]);
+        }
+        float evv[V], dvv[V], o[V];
+        er[u].get(evv);
+        dr[u].get(dvv);
+        double dot = 0.0;
+#pragma unroll
+        for (int c = 0; c < V; ++c) {
+          // σ'(y) = σ(y)·σ(-y) with σ(y) = e' (stored) and y = α z recomputed
+          const float dy = dvv[c] * evv[c] * __frcp_rn(1.f + ex2f_fast(a * z[c] * L2E));
+          dot = fma(double(dy), double(z[c]), dot);
+          o[c] = a * dy;
+        }
+#pragma unroll
+        for (int off = 16; off > 0; off >>= 1) dot += __shfl_xor_sync(0xffffffffu, dot, off);
+        store_row<V>(DZ + (k0 + kk) * D + lane * V, o);
+        if (lane == kk) dal_mine = float(dot);
+      }
+    }
+    if (lane < cnt) dalpha[k0 + lane] = dal_mine;
+  }
+}
+
 // e0[k] = edge_feat[in_eid[k]]  (a1)
 __global__ void permute_rows_kernel(const float *__restrict__ src, const int32_t *__restrict__ idx,
                                     int rows, int width, float *__restrict__ dst) {
@@ -999,25 +1085,43 @@ __global__ void head_bwd_reduce_kernel(const float *__restrict__ dy, const float
 
 // dh^L_u = dr_{graph(u)} / n_{graph(u)}
 // h_mask != null: emit dA = dh ⊙ LReLU'(A) (÷ deg for MEAN; sign(A) = sign(h)) instead of dh.
+// Thread = (node, 4 consecutive channels): float4 loads / stores, one node_graph lookup.
 __global__ void broadcast_dh_kernel(const float *__restrict__ dr, const int32_t *__restrict__ node_graph,
                                     const int32_t *__restrict__ node_off, int N, int D,
                                     const void *__restrict__ h_mask, int mask_bf,
                                     const int32_t *__restrict__ in_ptr,
                                     int mean, float slope, float *__restrict__ dh) {
-  const long total = long(N) * D;
+  const int D4 = D / 4;
+  const long total = long(N) * D4;
   for (long i = blockIdx.x * long(blockDim.x) + threadIdx.x; i < total;
        i += long(gridDim.x) * blockDim.x) {
-    const int u = int(i / D), k = int(i % D);
-    const int b = node_graph[u];
-    float v = dr[long(b) * D + k] / float(node_off[b + 1] - node_off[b]);
+    const int u = int(i / D4), k4 = int(i % D4);
+    const int b = __ldg(node_graph + u);
+    const float inv = 1.f / float(__ldg(node_off + b + 1) - __ldg(node_off + b));
+    const float4 r = __ldg(reinterpret_cast<const float4 *>(dr + long(b) * D) + k4);
+    float v[4] = {r.x * inv, r.y * inv, r.z * inv, r.w * inv};
     if (h_mask) {
-      v = v * lrelu_grad_from_out(mask_bf ? ld_act<true>(h_mask, i) : ld_act<false>(h_mask, i), slope);
+      float hm[4];
+      if (mask_bf) {
+        const uint2 x = __ldg(reinterpret_cast<const uint2 *>(reinterpret_cast<const uint16_t *>(h_mask) + long(u) * D) + k4);
+        hm[0] = __uint_as_float(x.x << 16); hm[1] = __uint_as_float(x.x & 0xFFFF0000u);
+        hm[2] = __uint_as_float(x.y << 16); hm[3] = __uint_as_float(x.y & 0xFFFF0000u);
+      } else {
+        const float4 x = __ldg(reinterpret_cast<const float4 *>(reinterpret_cast<const float *>(h_mask) + long(u) * D) + k4);
+        hm[0] = x.x; hm[1] = x.y; hm[2] = x.z; hm[3] = x.w;
+      }
+      float dsc = 1.f;
       if (mean) {
-        const int deg = in_ptr[u + 1] - in_ptr[u];
-        v = v / float(deg > 0 ? deg : 1);
+        const int deg = __ldg(in_ptr + u + 1) - __ldg(in_ptr + u);
+        dsc = float(deg > 0 ? deg : 1);
+      }
+#pragma unroll
+      for (int c = 0; c < 4; ++c) {
+        v[c] = v[c] * lrelu_grad_from_out(hm[c], slope);
+        if (mean) v[c] = v[c] / dsc;
       }
     }
-    dh[i] = v;
+    reinterpret_cast<float4 *>(dh + long(u) * D)[k4] = make_float4(v[0], v[1], v[2], v[3]);
   }
 }
 
@@ -1715,7 +1819,7 @@ int launch_head_backward(occu_ctx *ctx, const DevCsr &csr, const float *targets,
   LAUNCH_CHECK();
   OCCU_PROF_BEGIN(ctx, "broadcast_dh", st);
   const bool tcb = ctx->path != 1 && tc_supported(cf);    // TC backward consumes dA directly
-  broadcast_dh_kernel<<<grid_for(long(csr.N) * cf.d, 256, 8192), 256, 0, st>>>(
+  broadcast_dh_kernel<<<grid_for(long(csr.N) * cf.d / 4, 256, 16 * ctx->num_sms), 256, 0, st>>>(
       w.dr.as<float>(), csr.node_graph, csr.node_off, csr.N, cf.d,
       tcb ? w.h[cf.L - 1].ptr : nullptr, cf.prec == OCCU_BF16 ? 1 : 0, csr.in_ptr,
       cf.aggr == OCCU_AGGR_MEAN, cf.slope,
@@ -1784,18 +1888,21 @@ static int backward_layer_impl(occu_ctx *ctx, const DevCsr &csr, const BwdLayerA
       const int tiles = (csr.E + BM - 1) / BM;
       const int KS = a.Ke > D ? a.Ke : D;
       const size_t smB = (size_t(a.Ke) * D + BM * (KS + 4) + BM) * 4;
+      (void)tiles;
+      (void)smB;
+      // layer 1 only (Ke <= 16): e_in is the FP32 e0; e' is BF16 in OCCU_BF16
       OCCU_PROF_BEGIN(ctx, "edge_bwd_e", st);
-      if (bf) {    // layer 1 only (Ke <= 16): e_in is the FP32 e0, e' is BF16
-        set_smem(edge_bwd_e_kernel<D, true>, smB);
-        edge_bwd_e_kernel<D, true><<<grid_for(tiles, 1, sms), NT, smB, st>>>(
-            a.e_in, a.Ke, a.e, de, P + L.W_e[i], a.p, a.q, csr.in_src, csr.in_dst, csr.E,
-            w.DZ.as<float>(), w.dalpha.as<float>(), nullptr);
+      const int eg = grid_for((long(csr.E) + 31) / 32, NT / 32, 8 * sms);
+#define OCCU_EBS_ARGS a.e_in, a.Ke, a.e, de, P + L.W_e[i], a.p, a.q, csr.in_src, csr.in_dst, csr.E, \
+    w.DZ.as<float>(), w.dalpha.as<float>()
+      if (a.Ke <= 4) {
+        if (bf) edge_bwd_small_kernel<D, 4, true><<<eg, NT, 0, st>>>(OCCU_EBS_ARGS);
+        else edge_bwd_small_kernel<D, 4, false><<<eg, NT, 0, st>>>(OCCU_EBS_ARGS);
       } else {
-        set_smem(edge_bwd_e_kernel<D, false>, smB);
-        edge_bwd_e_kernel<D, false><<<grid_for(tiles, 1, sms), NT, smB, st>>>(
-            a.e_in, a.Ke, a.e, de, P + L.W_e[i], a.p, a.q, csr.in_src, csr.in_dst, csr.E,
-            w.DZ.as<float>(), w.dalpha.as<float>(), nullptr);
+        if (bf) edge_bwd_small_kernel<D, 16, true><<<eg, NT, 0, st>>>(OCCU_EBS_ARGS);
+        else edge_bwd_small_kernel<D, 16, false><<<eg, NT, 0, st>>>(OCCU_EBS_ARGS);
       }
+#undef OCCU_EBS_ARGS
       OCCU_PROF_END(ctx);
       LAUNCH_CHECK();
       ++n;

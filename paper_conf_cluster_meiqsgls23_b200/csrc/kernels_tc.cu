@@ -1644,8 +1644,10 @@ static bool encode_rows_map32_bf16(CUtensorMap *m, const void *A, long R, int K)
             CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
 
+// Bn < 16 or not a multiple of 16 (e.g. dW_e of layer 1, F_e = 4): the TMA box reads the
+// missing columns as zeros (out of bounds) and the MMA runs N = Bn rounded up to 16.
 bool wgrad_tc_supported(int A, int Bn) {
-  return A >= 32 && A <= 128 && A % 32 == 0 && Bn >= 16 && Bn <= 128 && Bn % 16 == 0;
+  return A >= 32 && A <= 128 && A % 32 == 0 && Bn >= 4 && Bn <= 128 && Bn % 4 == 0;
 }
 
 // partial must hold splits * A * Bn floats; returns the number of launches (1) or -err.
