@@ -1329,32 +1329,61 @@ __global__ void __launch_bounds__(NT) node_bwd_kernel(
   constexpr int V = D / 32;
   const int lane = threadIdx.x & 31;
   const int warps = (gridDim.x * NT) / 32;
-  float das[V], dad[V];
+  float das[V], dad[V], a_sv[V], a_dv[V];
 #pragma unroll
-  for (int c = 0; c < V; ++c) das[c] = dad[c] = 0.f;
+  for (int c = 0; c < V; ++c) {
+    das[c] = dad[c] = 0.f;
+    a_sv[c] = __ldg(a_s + lane * V + c);
+    a_dv[c] = __ldg(a_d + lane * V + c);
+  }
   for (int u = (blockIdx.x * NT + threadIdx.x) / 32; u < N; u += warps) {
     float acc[V];
 #pragma unroll
     for (int c = 0; c < V; ++c) acc[c] = 0.f;
     float dp = 0.f, dq = 0.f;
-    const int ob = out_ptr[u], oe = out_ptr[u + 1];
-    for (int j = ob; j < oe; ++j) {
-      const int k = out_pos[j];
-      const float *row = MG + long(k) * D + lane * V;
+    const int ob = __ldg(out_ptr + u), oe = __ldg(out_ptr + u + 1);
+    // out-edge rows four at a time, all loads in flight (indices clamped into the segment;
+    // surplus rows are never added), summed in ascending out-CSR order
+    constexpr int G = 4;
+    for (int j = ob; j < oe; j += G) {
+      int kk[G];
+      RawRow<V, false> rr[G];
+      float da[G];
 #pragma unroll
-      for (int c = 0; c < V; ++c) acc[c] += __ldg(row + c);
-      dp += __ldg(dalpha + k);
+      for (int u2 = 0; u2 < G; ++u2) kk[u2] = __ldg(out_pos + min(j + u2, oe - 1));
+#pragma unroll
+      for (int u2 = 0; u2 < G; ++u2) {
+        rr[u2].load(MG, long(kk[u2]), D, lane);
+        da[u2] = __ldg(dalpha + kk[u2]);
+      }
+#pragma unroll
+      for (int u2 = 0; u2 < G; ++u2) {
+        if (j + u2 < oe) {
+          float x[V];
+          rr[u2].get(x);
+#pragma unroll
+          for (int c = 0; c < V; ++c) acc[c] += x[c];
+          dp += da[u2];
+        }
+      }
     }
-    for (int k = in_ptr[u]; k < in_ptr[u + 1]; ++k) dq += __ldg(dalpha + k);
+    for (int k = __ldg(in_ptr + u); k < __ldg(in_ptr + u + 1); ++k) dq += __ldg(dalpha + k);
+    float hb[V], o[V];
+    {
+      RawRow<V, BF> hr;
+      hr.load(hbar, long(u), D, lane);
+      hr.get(hb);
+    }
 #pragma unroll
     for (int c = 0; c < V; ++c) {
       const int ch = lane * V + c;
-      const float v = acc[c] + dp * a_s[ch] + dq * a_d[ch];
-      const float hb = ld_act<BF>(hbar, long(u) * D + ch);
-      dP[long(u) * D + ch] = v * lrelu_grad_from_out(hb, slope);
-      das[c] = fmaf(dp, hb, das[c]);
-      dad[c] = fmaf(dq, hb, dad[c]);
+      const float v = acc[c] + dp * a_sv[c] + dq * a_dv[c];
+      o[c] = v * lrelu_grad_from_out(hb[c], slope);
+      das[c] = fmaf(dp, hb[c], das[c]);
+      dad[c] = fmaf(dq, hb[c], dad[c]);
+      (void)ch;
     }
+    store_row<V>(dP + long(u) * D + lane * V, o);
     if (lane == 0) {
       dpq[2 * long(u)] = dp;
       dpq[2 * long(u) + 1] = dq;
@@ -1488,6 +1517,41 @@ __global__ void __launch_bounds__(256) split_reduce_kernel(const float *__restri
     float t = 0.f;
     for (int j = 0; j < LANES; ++j) t += red[j][ol];
     out[o] = t;
+  }
+}
+
+// Several split-K reductions in one launch (the weight gradients of one layer and the
+// [da_s; da_d] partials): job j owns blocks [blk[j], blk[j+1]); within a job the order is
+// split_reduce_kernel's (fixed, deterministic).
+struct ReduceJob { const float *part; float *out; long n; int splits; int lanes = 8; };
+struct ReduceJobs { ReduceJob j[4]; int blk[5]; int count; };
+// job.lanes threads per output (8 for 128x128 weight gradients, 64 for the few outputs of
+// [da_s; da_d] with thousands of partials), 256 / lanes outputs per block.
+__global__ void __launch_bounds__(256) multi_reduce_kernel(const ReduceJobs jobs) {
+  __shared__ float red[256];
+  int q = 0;
+  while (q + 1 < jobs.count && int(blockIdx.x) >= jobs.blk[q + 1]) ++q;
+  const ReduceJob jb = jobs.j[q];
+  const int lanes = jb.lanes, opb = 256 / lanes;
+  const int ol = threadIdx.x % opb, l = threadIdx.x / opb;
+  const long o = long(int(blockIdx.x) - jobs.blk[q]) * opb + ol;
+  float a0 = 0.f, a1 = 0.f, a2 = 0.f, a3 = 0.f;     // four independent chains in flight
+  if (o < jb.n) {
+    int k = l;
+    for (; k + 3 * lanes < jb.splits; k += 4 * lanes) {
+      a0 += __ldg(jb.part + long(k) * jb.n + o);
+      a1 += __ldg(jb.part + long(k + lanes) * jb.n + o);
+      a2 += __ldg(jb.part + long(k + 2 * lanes) * jb.n + o);
+      a3 += __ldg(jb.part + long(k + 3 * lanes) * jb.n + o);
+    }
+    for (; k < jb.splits; k += lanes) a0 += __ldg(jb.part + long(k) * jb.n + o);
+  }
+  red[l * opb + ol] = (a0 + a1) + (a2 + a3);
+  __syncthreads();
+  if (l == 0 && o < jb.n) {
+    float t = 0.f;
+    for (int x = 0; x < lanes; ++x) t += red[x * opb + ol];
+    jb.out[o] = t;
   }
 }
 
@@ -1746,9 +1810,44 @@ static int reduce_splits(const occu_ctx *ctx, const float *part, int splits, lon
   return 1;
 }
 
+// Partial-sum slots of the deferred weight gradients: one per GEMM of a layer + the
+// [da_s; da_d] partials, each up to 2·148 splits x 128 x 128 floats.
+constexpr size_t WG_SLOT_FLOATS = size_t(2 * 160) * 128 * 128;
+
+static int launch_multi_reduce(const occu_ctx *ctx, ReduceJobs &rj, cudaStream_t st) {
+  if (rj.count == 0) return 0;
+  rj.blk[0] = 0;
+  for (int q = 0; q < rj.count; ++q) {
+    rj.j[q].lanes = rj.j[q].n >= 4096 ? 8 : 64;
+    const int opb = 256 / rj.j[q].lanes;
+    rj.blk[q + 1] = rj.blk[q] + int((rj.j[q].n + opb - 1) / opb);
+  }
+  OCCU_PROF_BEGIN(ctx, "split_reduce", st);
+  multi_reduce_kernel<<<rj.blk[rj.count], 256, 0, st>>>(rj);
+  OCCU_PROF_END(ctx);
+  LAUNCH_CHECK();
+  rj.count = 0;
+  return 1;
+}
+
+static int wgrad_impl(occu_ctx *ctx, const float *X, int A, const void *Yv, int Bn, long R,
+                      float *out, cudaStream_t st, bool ybf, ReduceJobs *defer, float *slot);
+
 // ybf: Y holds BF16 rows (OCCU_BF16 training); only the tensor-core kernel reads those.
 static int wgrad(occu_ctx *ctx, const float *X, int A, const void *Yv, int Bn, long R, float *out,
                  cudaStream_t st, bool ybf = false) {
+  return wgrad_impl(ctx, X, A, Yv, Bn, R, out, st, ybf, nullptr, nullptr);
+}
+
+// Deferred: the partials go to `slot` and the reduction is appended to `rj` (one
+// launch_multi_reduce per layer instead of one reduction launch per GEMM).
+static int wgrad_deferred(occu_ctx *ctx, const float *X, int A, const void *Yv, int Bn, long R,
+                          float *out, cudaStream_t st, bool ybf, ReduceJobs &rj, float *slot) {
+  return wgrad_impl(ctx, X, A, Yv, Bn, R, out, st, ybf, &rj, slot);
+}
+
+static int wgrad_impl(occu_ctx *ctx, const float *X, int A, const void *Yv, int Bn, long R,
+                      float *out, cudaStream_t st, bool ybf, ReduceJobs *defer, float *slot) {
   const float *Y = reinterpret_cast<const float *>(Yv);
   const long n = long(A) * Bn;
   const int ta = (A + 127) / 128, tb = (Bn + 127) / 128;
@@ -1759,35 +1858,43 @@ static int wgrad(occu_ctx *ctx, const float *X, int A, const void *Yv, int Bn, l
   }
   if (ybf && !wgrad_tc_supported(A, Bn)) return -int(cudaErrorInvalidValue);
   static const long tc_min = getenv("OCCU_WGRAD_TC_MIN") ? atol(getenv("OCCU_WGRAD_TC_MIN")) : 4096;
+  auto get_part = [&](int sp) -> float * {
+    if (defer) return slot;
+    if (ctx->ws.partial.ensure(size_t(sp) * n * 4) != cudaSuccess) return nullptr;
+    return ctx->ws.partial.as<float>();
+  };
+  auto finish = [&](float *part, int sp) -> int {
+    if (defer) {
+      defer->j[defer->count++] = ReduceJob{part, out, n, sp};
+      return 0;
+    }
+    return reduce_splits(ctx, part, sp, n, out, st);
+  };
   if (ctx->path != 1 && wgrad_tc_supported(A, Bn) && (R >= tc_min || ybf)) {
     const int sp = ctx->num_sms;
-    if (ctx->ws.partial.ensure(size_t(sp) * n * 4) != cudaSuccess) return -int(cudaErrorMemoryAllocation);
-    float *part = ctx->ws.partial.as<float>();
+    float *part = get_part(sp);
+    if (!part) return -int(cudaErrorMemoryAllocation);
     int r = launch_wgrad_tc(ctx, X, A, Yv, Bn, R, sp, part, st, ybf);
     if (r < 0) return r;
-    return r + reduce_splits(ctx, part, sp, n, out, st);
+    return r + finish(part, sp);
   }
   if (n <= 2 * NT && A <= 128 && Bn <= 128) {
     const int sp = 2 * ctx->num_sms;
-    if (ctx->ws.partial.ensure(size_t(sp) * n * 4) != cudaSuccess) return -int(cudaErrorMemoryAllocation);
-    float *part = ctx->ws.partial.as<float>();
+    float *part = get_part(sp);
+    if (!part) return -int(cudaErrorMemoryAllocation);
     OCCU_PROF_BEGIN(ctx, "wgrad_skinny", st);
     wgrad_skinny_kernel<<<sp, NT, 0, st>>>(X, A, Y, Bn, R, sp, part);
     OCCU_PROF_END(ctx);
     LAUNCH_CHECK();
-    return 1 + reduce_splits(ctx, part, sp, n, out, st);
+    return 1 + finish(part, sp);
   }
-  if (ctx->ws.partial.ensure(size_t(splits) * n * 4) != cudaSuccess) return -int(cudaErrorMemoryAllocation);
-  float *part = ctx->ws.partial.as<float>();
+  float *part = get_part(splits);
+  if (!part) return -int(cudaErrorMemoryAllocation);
   OCCU_PROF_BEGIN(ctx, "wgrad_partial", st);
   wgrad_partial_kernel<<<dim3(splits, ta, tb), NT, 0, st>>>(X, A, Y, Bn, R, splits, part);
   OCCU_PROF_END(ctx);
   LAUNCH_CHECK();
-  OCCU_PROF_BEGIN(ctx, "wgrad_reduce", st);
-  wgrad_reduce_kernel<<<grid_for(n, 256, 1024), 256, 0, st>>>(part, splits, n, out);
-  OCCU_PROF_END(ctx);
-  LAUNCH_CHECK();
-  return 2;
+  return 1 + finish(part, splits);
 }
 
 int launch_wgrad(occu_ctx *ctx, const float *X, int A, const void *Y, int Bn, long R, float *out,
@@ -1952,16 +2059,21 @@ static int backward_layer_impl(occu_ctx *ctx, const DevCsr &csr, const BwdLayerA
   OCCU_PROF_END(ctx);
   LAUNCH_CHECK();
   ++n;
-  if (tc) {
-    if ((r = reduce_splits(ctx, da_part, nb_blocks, 2 * D, G + L.a_s[i], st)) < 0) return r;
-    n += r;
-  }
-  // dW_m = DVᵀ E' ; dW_e = DZᵀ E_in ; dW_u = dPᵀ H_in ; [da_s; da_d] = [dp dq]ᵀ h̄
-  if ((r = wgrad(ctx, w.DV.as<float>(), D, a.e, D, csr.E, G + L.W_m[i], st, bf)) < 0) return r;
+  // dW_m = DVᵀ E' ; dW_e = DZᵀ E_in ; dW_u = dPᵀ H_in ; [da_s; da_d] = [dp dq]ᵀ h̄ — partial
+  // sums into per-GEMM slots, all of the layer's split reductions in one launch
+  ReduceJobs rj{};
+  if (tc) rj.j[rj.count++] = ReduceJob{da_part, G + L.a_s[i], long(2 * D), nb_blocks};
+  if (w.partial.ensure(3 * WG_SLOT_FLOATS * 4) != cudaSuccess) return -int(cudaErrorMemoryAllocation);
+  float *slot = w.partial.as<float>();
+  if ((r = wgrad_deferred(ctx, w.DV.as<float>(), D, a.e, D, csr.E, G + L.W_m[i], st, bf, rj, slot)) < 0) return r;
   n += r;
-  if ((r = wgrad(ctx, w.DZ.as<float>(), D, a.e_in, a.Ke, csr.E, G + L.W_e[i], st, in_bf)) < 0) return r;
+  if ((r = wgrad_deferred(ctx, w.DZ.as<float>(), D, a.e_in, a.Ke, csr.E, G + L.W_e[i], st, in_bf, rj,
+                          slot + WG_SLOT_FLOATS)) < 0) return r;
   n += r;
-  if ((r = wgrad(ctx, w.dP.as<float>(), D, a.h_in, a.K, csr.N, G + L.W_u[i], st, in_bf)) < 0) return r;
+  if ((r = wgrad_deferred(ctx, w.dP.as<float>(), D, a.h_in, a.K, csr.N, G + L.W_u[i], st, in_bf, rj,
+                          slot + 2 * WG_SLOT_FLOATS)) < 0) return r;
+  n += r;
+  if ((r = launch_multi_reduce(ctx, rj, st)) < 0) return r;
   n += r;
   if (!tc) {
     if ((r = wgrad(ctx, w.dpq.as<float>(), 2, a.hbar, D, csr.N, G + L.a_s[i], st)) < 0) return r;
