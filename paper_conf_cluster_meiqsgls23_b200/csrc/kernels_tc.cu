@@ -1363,7 +1363,13 @@ __global__ void __launch_bounds__(256) edge_small_kernel(
 // YBF (OCCU_BF16 training, R28): Y rows are BF16.  TMA lands them (32 rows x 64 bf16 SW128
 // boxes) in the Y-lo region; the lo warps widen them (exactly) into the Y raw region, and
 // since a BF16 value is its own tf32 hi part (Y lo = 0) the X_hi·Y_lo product is skipped.
-constexpr int WG_NS = 3;                  // pipeline stages of 32 rows
+constexpr int WG_ROWS = 32;               // rows (K) per pipeline stage
+constexpr int WG_NS = 3;                  // pipeline stages (16-row x 6 and 2 CTAs/SM measured slower)
+constexpr int WG_BOX = WG_ROWS * 128;     // one TMA box: WG_ROWS rows x 32 fp32 (or 64 bf16)
+constexpr int WG_REG = 4 * WG_BOX;        // one operand region (4 boxes = 128 columns)
+constexpr int WG_STAGE = 4 * WG_REG;      // X raw, X lo, Y raw, Y lo
+constexpr int WG_Q4 = WG_ROWS * 8;        // float4 per box
+constexpr int WG_IT = 2 * 4 * WG_Q4 / 256;  // float4 per lo-warp thread per stage
 constexpr int WG_NTH = 320;               // warp0 TMA, warp1 MMA, warps 2-9 lo / epilogue
 
 // Logical 16-byte chunk stored at physical slot pc of 128-byte row r under the TMA
@@ -1379,16 +1385,17 @@ wgrad_tc_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant_
   extern __shared__ uint8_t smem_raw[];
   const uint32_t sa = tc::smem_u32(smem_raw);
   uint8_t *base = smem_raw + ((1024 - (sa & 1023)) & 1023);
-  // stage s: X raw (4 boxes x 4 KB), X lo, Y raw, Y lo
-  auto stage = [&](int s2) { return base + s2 * 65536; };
-  uint64_t *bars = reinterpret_cast<uint64_t *>(base + WG_NS * 65536);
+  // stage s: X raw (4 boxes of WG_ROWS rows x 128 B), X lo, Y raw, Y lo (Y-lo region = BF16
+  // landing zone when YBF)
+  auto stage = [&](int s2) { return base + s2 * WG_STAGE; };
+  uint64_t *bars = reinterpret_cast<uint64_t *>(base + WG_NS * WG_STAGE);
   uint64_t *full = bars, *lo_ready = bars + WG_NS, *empty = bars + 2 * WG_NS, *done = bars + 3 * WG_NS;
   uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(bars + 3 * WG_NS + 1);
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int nbx = (A + 31) / 32, nby = (Bn + 31) / 32, nbyb = (Bn + 63) / 64;
   const int Npad = (Bn + 15) / 16 * 16;
   // zero every box region once: boxes that TMA never writes (A or B < 128) stay zero
-  for (int i = threadIdx.x; i < WG_NS * 65536 / 16; i += WG_NTH)
+  for (int i = threadIdx.x; i < WG_NS * WG_STAGE / 16; i += WG_NTH)
     reinterpret_cast<float4 *>(base)[i] = make_float4(0.f, 0.f, 0.f, 0.f);
   if (threadIdx.x == 0) {
     for (int j = 0; j < WG_NS; ++j) {
@@ -1407,7 +1414,7 @@ wgrad_tc_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant_
   const uint32_t tmem = *tmem_slot;
   const long per = (R + splits - 1) / splits;
   const long rb = blockIdx.x * per, re = min(R, rb + per);
-  const int nst = rb < re ? int((re - rb + 31) / 32) : 0;
+  const int nst = rb < re ? int((re - rb + WG_ROWS - 1) / WG_ROWS) : 0;
 
   if (warp == 0) {
     if (lane == 0) {
@@ -1416,14 +1423,14 @@ wgrad_tc_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant_
       for (int i = 0; i < nst; ++i) {
         const int j = i % WG_NS;
         if (i >= WG_NS) tc::mbar_wait(empty + j, ((i / WG_NS) - 1) & 1);
-        const int r0 = int(rb + long(i) * 32);
+        const int r0 = int(rb + long(i) * WG_ROWS);
         uint8_t *st = stage(j);
-        tc::mbar_arrive_expect_tx(full + j, uint32_t(nbx + (YBF ? nbyb : nby)) * 4096u);
-        for (int b = 0; b < nbx; ++b) tc::tma_load_2d(st + b * 4096, &xmap, 32 * b, r0, full + j);
+        tc::mbar_arrive_expect_tx(full + j, uint32_t(nbx + (YBF ? nbyb : nby)) * uint32_t(WG_BOX));
+        for (int b = 0; b < nbx; ++b) tc::tma_load_2d(st + b * WG_BOX, &xmap, 32 * b, r0, full + j);
         if (YBF)
-          for (int b = 0; b < nbyb; ++b) tc::tma_load_2d(st + 49152 + b * 4096, &ymap, 64 * b, r0, full + j);
+          for (int b = 0; b < nbyb; ++b) tc::tma_load_2d(st + 3 * WG_REG + b * WG_BOX, &ymap, 64 * b, r0, full + j);
         else
-          for (int b = 0; b < nby; ++b) tc::tma_load_2d(st + 32768 + b * 4096, &ymap, 32 * b, r0, full + j);
+          for (int b = 0; b < nby; ++b) tc::tma_load_2d(st + 2 * WG_REG + b * WG_BOX, &ymap, 32 * b, r0, full + j);
       }
     }
     __syncwarp();
@@ -1435,11 +1442,11 @@ wgrad_tc_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant_
       tc::fence_after_sync();
       if (lane == 0) {
         const uint32_t st = tc::smem_u32(stage(j));
-        for (int kg = 0; kg < 4; ++kg) {
-          const uint64_t ah = tc::sdesc_sw128b32_mn(st + kg * 1024, 4096);
-          const uint64_t al = tc::sdesc_sw128b32_mn(st + 16384 + kg * 1024, 4096);
-          const uint64_t bh = tc::sdesc_sw128b32_mn(st + 32768 + kg * 1024, 4096);
-          const uint64_t bl = tc::sdesc_sw128b32_mn(st + 49152 + kg * 1024, 4096);
+        for (int kg = 0; kg < WG_ROWS / 8; ++kg) {
+          const uint64_t ah = tc::sdesc_sw128b32_mn(st + kg * 1024, WG_BOX);
+          const uint64_t al = tc::sdesc_sw128b32_mn(st + WG_REG + kg * 1024, WG_BOX);
+          const uint64_t bh = tc::sdesc_sw128b32_mn(st + 2 * WG_REG + kg * 1024, WG_BOX);
+          const uint64_t bl = tc::sdesc_sw128b32_mn(st + 3 * WG_REG + kg * 1024, WG_BOX);
           tc::mma_tf32_ss(tmem, ah, bh, idsc, (i > 0 || kg > 0) ? 1u : 0u);
           if (!YBF) tc::mma_tf32_ss(tmem, ah, bl, idsc, 1u);
           tc::mma_tf32_ss(tmem, al, bh, idsc, 1u);
@@ -1455,13 +1462,13 @@ wgrad_tc_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant_
       const int j = i % WG_NS;
       tc::mbar_wait(full + j, (i / WG_NS) & 1);
       uint8_t *st = stage(j);
-      const long r0 = rb + long(i) * 32;
+      const long r0 = rb + long(i) * WG_ROWS;
       // X raw -> X lo (boxes 0..nbx), Y raw -> Y lo; rows beyond this CTA's range -> 0.
-      // 2 operands x 4 boxes x 256 float4 = 8 per thread, all loads issued before use.
-      float4 v[8];
+      // 2 operands x 4 boxes x WG_ROWS·8 float4 = WG_IT per thread, all loads issued first.
+      float4 v[WG_IT];
 #pragma unroll
-      for (int it = 0; it < 8; ++it) {
-        const int f = t + it * 256, op = f >> 10, b = (f >> 8) & 3, q4 = f & 255;
+      for (int it = 0; it < WG_IT; ++it) {
+        const int f = t + it * 256, op = f / (4 * WG_Q4), b = (f / WG_Q4) & 3, q4 = f % WG_Q4;
         v[it] = make_float4(0.f, 0.f, 0.f, 0.f);
         if (b < (op == 0 ? nbx : nby)) {
           if (YBF && op == 1) {
@@ -1469,35 +1476,35 @@ wgrad_tc_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant_
             // logical chunk c (columns 32b+4c..+3) <- bf16 box b/2 (plain SW128: chunk ^ (row & 7)),
             // logical chunk 4(b&1) + c/2, half c&1
             const int rr = q4 >> 3, c = wg_logical_chunk(q4 & 7, rr), cb = 4 * (b & 1) + (c >> 1);
-            const uint2 w = *reinterpret_cast<const uint2 *>(st + 49152 + (b >> 1) * 4096 + rr * 128 +
+            const uint2 w = *reinterpret_cast<const uint2 *>(st + 3 * WG_REG + (b >> 1) * WG_BOX + rr * 128 +
                                                              ((cb ^ (rr & 7)) << 4) + (c & 1) * 8);
             v[it] = make_float4(__uint_as_float(w.x << 16), __uint_as_float(w.x & 0xFFFF0000u),
                                 __uint_as_float(w.y << 16), __uint_as_float(w.y & 0xFFFF0000u));
           } else {
-            v[it] = reinterpret_cast<const float4 *>(st + op * 32768 + b * 4096)[q4];
+            v[it] = reinterpret_cast<const float4 *>(st + op * 2 * WG_REG + b * WG_BOX)[q4];
           }
         }
       }
 #pragma unroll
-      for (int it = 0; it < 8; ++it) {
-        const int f = t + it * 256, op = f >> 10, b = (f >> 8) & 3, q4 = f & 255;
+      for (int it = 0; it < WG_IT; ++it) {
+        const int f = t + it * 256, op = f / (4 * WG_Q4), b = (f / WG_Q4) & 3, q4 = f % WG_Q4;
         if (b >= (op == 0 ? nbx : nby)) continue;
         float4 x = v[it];
         if (YBF && op == 1) {                             // widened BF16 row: raw, no lo
           if (r0 + (q4 >> 3) >= re) x = make_float4(0.f, 0.f, 0.f, 0.f);
-          reinterpret_cast<float4 *>(st + 32768 + b * 4096)[q4] = x;
+          reinterpret_cast<float4 *>(st + 2 * WG_REG + b * WG_BOX)[q4] = x;
           continue;
         }
         if (r0 + (q4 >> 3) >= re) {                       // 8 float4 per 128-byte row
           x = make_float4(0.f, 0.f, 0.f, 0.f);
-          reinterpret_cast<float4 *>(st + op * 32768 + b * 4096)[q4] = x;
+          reinterpret_cast<float4 *>(st + op * 2 * WG_REG + b * WG_BOX)[q4] = x;
         }
         float4 l;
         l.x = x.x - __uint_as_float(__float_as_uint(x.x) & 0xFFFFE000u);
         l.y = x.y - __uint_as_float(__float_as_uint(x.y) & 0xFFFFE000u);
         l.z = x.z - __uint_as_float(__float_as_uint(x.z) & 0xFFFFE000u);
         l.w = x.w - __uint_as_float(__float_as_uint(x.w) & 0xFFFFE000u);
-        reinterpret_cast<float4 *>(st + op * 32768 + 16384 + b * 4096)[q4] = l;
+        reinterpret_cast<float4 *>(st + op * 2 * WG_REG + WG_REG + b * WG_BOX)[q4] = l;
       }
       asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
       tc::mbar_arrive(lo_ready + j);
@@ -1617,7 +1624,7 @@ static bool encode_rows_map32(CUtensorMap *m, const float *A, long R, int K) {
   }
   const cuuint64_t dims[2] = {cuuint64_t(K), cuuint64_t(R)};
   const cuuint64_t strides[1] = {cuuint64_t(K) * 4};
-  const cuuint32_t box[2] = {32, 32};
+  const cuuint32_t box[2] = {32, WG_ROWS};
   const cuuint32_t estr[2] = {1, 1};
   return fn(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, const_cast<float *>(A), dims, strides, box, estr,
             CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B,
@@ -1637,7 +1644,7 @@ static bool encode_rows_map32_bf16(CUtensorMap *m, const void *A, long R, int K)
   }
   const cuuint64_t dims[2] = {cuuint64_t(K), cuuint64_t(R)};
   const cuuint64_t strides[1] = {cuuint64_t(K) * 2};
-  const cuuint32_t box[2] = {64, 32};
+  const cuuint32_t box[2] = {64, WG_ROWS};
   const cuuint32_t estr[2] = {1, 1};
   return fn(m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void *>(A), dims, strides, box, estr,
             CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
@@ -1657,7 +1664,7 @@ int launch_wgrad_tc(const occu_ctx *ctx, const float *X, int A, const void *Y, i
   if (!encode_rows_map32(&xm, X, R, A) ||
       !(ybf ? encode_rows_map32_bf16(&ym, Y, R, Bn) : encode_rows_map32(&ym, static_cast<const float *>(Y), R, Bn)))
     return -int(cudaErrorInvalidValue);
-  const size_t smem = 1024 + WG_NS * 65536 + 256;
+  const size_t smem = 1024 + size_t(WG_NS) * WG_STAGE + 256;
   OCCU_PROF_BEGIN(ctx, "wgrad_tc", st);
   if (ybf) {
     set_smem(wgrad_tc_kernel<true>, smem);
