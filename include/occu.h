@@ -138,6 +138,19 @@ void occu_batch_free(occu_csr_batch *b);
 occu_status occu_predict(occu_ctx *ctx, const occu_csr_batch *csr_batch,
                          const float *node_feat, const float *edge_feat, float *out_occ);
 
+/* Pipelined variant for a stream of host batches: returns at once.  The batch's CSR and
+ * features are copied on an internal copy stream into one of two device staging slots while
+ * the previous batch still computes on the ctx stream; the forward waits for its copy, and
+ * out_occ (host, pinned for overlap) is written by an async D2H on the ctx stream.  The call
+ * blocks only until the previous call's copy has landed, so the caller keeps csr_batch,
+ * node_feat and edge_feat alive and unmodified until the next occu_predict_async (or
+ * occu_wait) returns, and reads out_occ after occu_wait.  EINVAL for device pointers or a device
+ * batch (use occu_predict, which is already stream-ordered for those). */
+occu_status occu_predict_async(occu_ctx *ctx, const occu_csr_batch *csr_batch,
+                               const float *node_feat, const float *edge_feat, float *out_occ);
+/* Blocks until every occu_predict_async issued on ctx has completed. */
+occu_status occu_wait(occu_ctx *ctx);
+
 /* ---- training (P209-P213, P273) ------------------------------------------- */
 /* Forward with saved activations, MSE loss scaled by 1/global_num_graphs,
  * backward, NCCL allreduce of the flat gradient (if occu_dist_init was

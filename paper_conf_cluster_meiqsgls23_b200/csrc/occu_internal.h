@@ -51,6 +51,7 @@ struct Workspace {
   DevBuf dy, dc, dr, dh, dhprev, dP, MG, DV, DZ, deA, deB, dalpha, dpq, partial, loss;
   DevBuf tcpart;           // tensor-core aggregation: boundary-segment partials
   DevBuf dpart;            // per-warp [da_s; da_d] partials
+  DevBuf anf[2], aef[2], acsr[2];   // occu_predict_async: double-buffered input staging
   void release_all();
 };
 
@@ -108,6 +109,10 @@ struct occu_ctx {
   bool h_last_stored = true;   // false: the last forward kept only readout partials of h_L
   int64_t launches = 0;
   mutable occu::Profiler prof;
+  // occu_predict_async: H2D on a copy stream into staging slot a_slot, compute on `stream`
+  cudaStream_t copy_stream = nullptr;
+  cudaEvent_t a_copied[2] = {nullptr, nullptr}, a_free[2] = {nullptr, nullptr};
+  int a_slot = 0;
   // data parallel
   ncclComm *comm = nullptr;
   int rank = 0, world = 1;

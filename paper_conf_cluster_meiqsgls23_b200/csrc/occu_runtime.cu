@@ -46,9 +46,10 @@ void DevBuf::release() {
 void Workspace::release_all() {
   DevBuf *bufs[] = {&node_feat, &edge_feat, &targets, &out_occ, &csr, &e0, &g, &r, &c, &yhat,
                     &dy, &dc, &dr, &dh, &dhprev, &dP, &MG, &DV, &DZ, &deA, &deB, &dalpha,
-                    &dpq, &partial, &loss, &tcpart, &dpart};
+                    &dpq, &partial, &loss, &tcpart, &dpart, &rpart, &anf[0], &anf[1],
+                    &aef[0], &aef[1], &acsr[0], &acsr[1]};
   for (DevBuf *b : bufs) b->release();
-  for (auto *v : {&hbar, &p, &q, &e, &h})
+  for (auto *v : {&hbar, &p, &q, &e, &h, &gs})
     for (DevBuf &b : *v) b.release();
 }
 
@@ -165,8 +166,12 @@ occu_status validate_cfg(const occu_config *c) {
   return OCCU_OK;
 }
 
-// Device view of the batch (copies a host batch into the workspace).
+// Device view of the batch (copies a host batch into `dst` on stream `s`).
+occu_status upload_csr(occu_ctx *ctx, const occu_csr_batch *b, DevBuf &dst, cudaStream_t s, DevCsr &out);
 occu_status resolve_csr(occu_ctx *ctx, const occu_csr_batch *b, DevCsr &out) {
+  return upload_csr(ctx, b, ctx->ws.csr, ctx->stream, out);
+}
+occu_status upload_csr(occu_ctx *ctx, const occu_csr_batch *b, DevBuf &dst, cudaStream_t s, DevCsr &out) {
   if (!b) return fail(ctx, OCCU_EINVAL, "csr_batch is NULL");
   out.B = b->num_graphs;
   out.N = b->num_nodes;
@@ -179,8 +184,8 @@ occu_status resolve_csr(occu_ctx *ctx, const occu_csr_batch *b, DevCsr &out) {
   }
   const size_t B1 = out.B + 1, N1 = out.N + 1, E = out.E, N = out.N;
   const size_t total = 2 * B1 + 2 * N1 + 4 * E + N;
-  CK(ctx->ws.csr.ensure(total * 4), "csr alloc");
-  int32_t *d = ctx->ws.csr.as<int32_t>();
+  CK(dst.ensure(total * 4), "csr alloc");
+  int32_t *d = dst.as<int32_t>();
   int32_t *q = d;
   const int32_t *srcs[9] = {b->node_off, b->edge_off, b->in_ptr, b->out_ptr, b->in_src,
                             b->in_dst, b->in_eid, b->out_pos, b->node_graph};
@@ -189,11 +194,11 @@ occu_status resolve_csr(occu_ctx *ctx, const occu_csr_batch *b, DevCsr &out) {
                              &out.in_dst, &out.in_eid, &out.out_pos, &out.node_graph};
   if (b->priv == static_cast<void *>(b->node_off)) {
     // occu_pack output: one contiguous allocation in this order -> a single copy
-    CK(cudaMemcpyAsync(d, b->node_off, total * 4, cudaMemcpyHostToDevice, ctx->stream), "csr H2D");
+    CK(cudaMemcpyAsync(d, b->node_off, total * 4, cudaMemcpyHostToDevice, s), "csr H2D");
     for (int i = 0; i < 9; ++i) { *dsts[i] = q; q += lens[i]; }
   } else {
     for (int i = 0; i < 9; ++i) {
-      if (lens[i]) CK(cudaMemcpyAsync(q, srcs[i], lens[i] * 4, cudaMemcpyHostToDevice, ctx->stream), "csr H2D");
+      if (lens[i]) CK(cudaMemcpyAsync(q, srcs[i], lens[i] * 4, cudaMemcpyHostToDevice, s), "csr H2D");
       *dsts[i] = q;
       q += lens[i];
     }
@@ -433,6 +438,14 @@ occu_status occu_destroy(occu_ctx *ctx) {
   cudaSetDevice(ctx->device);
   cudaStreamSynchronize(ctx->stream);
   if (ctx->comm) ncclCommDestroy(ctx->comm);
+  if (ctx->copy_stream) {
+    cudaStreamSynchronize(ctx->copy_stream);
+    cudaStreamDestroy(ctx->copy_stream);
+    for (int k = 0; k < 2; ++k) {
+      cudaEventDestroy(ctx->a_copied[k]);
+      cudaEventDestroy(ctx->a_free[k]);
+    }
+  }
   ctx->ws.release_all();
   ctx->params.release();
   ctx->wimg.release();
@@ -570,6 +583,58 @@ occu_status occu_predict(occu_ctx *ctx, const occu_csr_batch *csr_batch, const f
     CK(cudaMemcpyAsync(out_occ, ctx->ws.yhat.ptr, ob, cudaMemcpyDeviceToDevice, ctx->stream), "D2D");
   }
   CK(cudaGetLastError(), "predict");
+  return OCCU_OK;
+}
+
+occu_status occu_predict_async(occu_ctx *ctx, const occu_csr_batch *csr_batch,
+                               const float *node_feat, const float *edge_feat, float *out_occ) {
+  occu_status st = check_ready(ctx);
+  if (st != OCCU_OK) return st;
+  if (!csr_batch || !node_feat || !out_occ || (csr_batch->num_edges > 0 && !edge_feat))
+    return fail(ctx, OCCU_EINVAL, "NULL argument");
+  if (csr_batch->on_device || is_device_ptr(node_feat) || is_device_ptr(out_occ))
+    return fail(ctx, OCCU_EINVAL, "occu_predict_async takes a host batch and host (pinned) buffers");
+  if (!ctx->copy_stream) {
+    CK(cudaStreamCreateWithFlags(&ctx->copy_stream, cudaStreamNonBlocking), "copy stream");
+    for (int k = 0; k < 2; ++k) {
+      CK(cudaEventCreateWithFlags(&ctx->a_copied[k], cudaEventDisableTiming), "event");
+      CK(cudaEventCreateWithFlags(&ctx->a_free[k], cudaEventDisableTiming), "event");
+    }
+  }
+  ctx->launches = 0;
+  const int slot = ctx->a_slot;
+  ctx->a_slot ^= 1;
+  // the previous call's host inputs become reusable once its copy has landed: the host
+  // waits here (the copy is the pipeline's slowest stage, so this costs no throughput)
+  CK(cudaEventSynchronize(ctx->a_copied[slot ^ 1]), "wait previous copy");
+  const occu_config &c = ctx->cfg;
+  Workspace &w = ctx->ws;
+  // the slot's buffers are reused only after the forward that read them has finished
+  CK(cudaStreamWaitEvent(ctx->copy_stream, ctx->a_free[slot], 0), "wait slot");
+  DevCsr csr;
+  if ((st = upload_csr(ctx, csr_batch, w.acsr[slot], ctx->copy_stream, csr)) != OCCU_OK) return st;
+  CK(w.anf[slot].ensure(size_t(csr.N) * c.F_n * 4), "alloc node_feat");
+  CK(w.aef[slot].ensure(std::max<size_t>(size_t(csr.E) * c.F_e * 4, 4)), "alloc edge_feat");
+  CK(cudaMemcpyAsync(w.anf[slot].ptr, node_feat, size_t(csr.N) * c.F_n * 4, cudaMemcpyHostToDevice,
+                     ctx->copy_stream), "node_feat H2D");
+  if (csr.E > 0)
+    CK(cudaMemcpyAsync(w.aef[slot].ptr, edge_feat, size_t(csr.E) * c.F_e * 4, cudaMemcpyHostToDevice,
+                       ctx->copy_stream), "edge_feat H2D");
+  CK(cudaEventRecord(ctx->a_copied[slot], ctx->copy_stream), "record");
+  CK(cudaStreamWaitEvent(ctx->stream, ctx->a_copied[slot], 0), "wait copy");
+  if ((st = forward(ctx, csr, w.anf[slot].as<float>(), w.aef[slot].as<float>(), ctx->keep)) != OCCU_OK)
+    return st;
+  CK(cudaEventRecord(ctx->a_free[slot], ctx->stream), "record");
+  CK(cudaMemcpyAsync(out_occ, w.yhat.ptr, size_t(csr.B) * 4, cudaMemcpyDeviceToHost, ctx->stream), "D2H");
+  CK(cudaGetLastError(), "predict_async");
+  return OCCU_OK;
+}
+
+occu_status occu_wait(occu_ctx *ctx) {
+  if (!ctx) return fail(nullptr, OCCU_EINVAL, "ctx is NULL");
+  CK(cudaSetDevice(ctx->device), "cudaSetDevice");
+  if (ctx->copy_stream) CK(cudaStreamSynchronize(ctx->copy_stream), "sync");
+  CK(cudaStreamSynchronize(ctx->stream), "sync");
   return OCCU_OK;
 }
 

@@ -92,6 +92,8 @@ def lib():
             "occu_batch_to_device": ([VP, P(CsrBatch), P(P(CsrBatch))], I32),
             "occu_batch_free": ([P(CsrBatch)], None),
             "occu_predict": ([VP, P(CsrBatch), VP, VP, VP], I32),
+            "occu_predict_async": ([VP, P(CsrBatch), VP, VP, VP], I32),
+            "occu_wait": ([VP], I32),
             "occu_train_step": ([VP, P(BatchStruct), VP, C.c_float, P(C.c_float)], I32),
             "occu_compute_grads": ([VP, P(BatchStruct), VP, P(C.c_float)], I32),
             "occu_get_grads": ([VP, VP, SZ], I32),
@@ -253,6 +255,7 @@ class Model:
 
     def __init__(self, cfg: Config, device: int = 0, stream=None):
         self.cfg = cfg
+        self._inflight = []
         self._ctx = C.c_void_p()
         if stream is None:
             try:
@@ -333,6 +336,22 @@ class Model:
         op, _, k3 = _ptr(out)
         _check(lib().occu_predict(self._ctx, csr._p, nf, ef, op), self._ctx)
         return out
+
+    def predict_async(self, csr: Csr, node_feat, edge_feat, out):
+        """occu_predict_async: host batch, pinned host features and output; returns at once.
+        The arguments are kept referenced until wait() (the library reads them later)."""
+        nf, dev, k1 = _ptr(node_feat)
+        ef, _, k2 = _ptr(edge_feat)
+        op, _, k3 = _ptr(out)
+        _check(lib().occu_predict_async(self._ctx, csr._p, nf, ef, op), self._ctx)
+        # the previous call's inputs are free once this call returns; outputs until wait()
+        self._inflight = [x for x in self._inflight if x[0] is None] + [(csr, k1, k2, k3, node_feat, edge_feat, out)]
+        self._inflight = [(None, None, None, None, None, None, x[6]) for x in self._inflight[:-1]] + self._inflight[-1:]
+        return out
+
+    def wait(self):
+        _check(lib().occu_wait(self._ctx), self._ctx)
+        self._inflight.clear()
 
     def _batch(self, csr, node_feat, edge_feat, global_num_graphs):
         nf, _, k1 = _ptr(node_feat)

@@ -357,3 +357,29 @@ def test_cfg3_full_size_training_properties():
     # every parameter tensor receives a gradient (the identity above holds trivially for 0)
     for k, v in weights.unflatten(wcfg(c), g_full).items():
         assert np.linalg.norm(v) > 0, k
+
+
+def test_predict_async_pipeline_matches_predict():
+    """occu_predict_async over a stream of different host batches (double-buffered staging,
+    copy stream): every batch's predictions are bitwise those of the blocking occu_predict,
+    and misuse (device inputs) is rejected."""
+    import torch
+    c = mk(3, 128)
+    m = occu.Model(c)
+    m.init_weights(5)
+    batches = [configs.random_dag_batch(30 + 7 * k, 1200 + k, max_nodes=60, hub=True) for k in range(5)]
+    want = [m.predict(occu.pack(b.graphs), b.node_feat, b.edge_feat) for b in batches]
+    pins = [(torch.from_numpy(b.node_feat).pin_memory(), torch.from_numpy(b.edge_feat).pin_memory(),
+             torch.empty(b.num_graphs, dtype=torch.float32).pin_memory()) for b in batches]
+    for rep in range(2):
+        for b, (nf, ef, out) in zip(batches, pins):
+            out.fill_(float("nan"))
+            m.predict_async(occu.pack(b.graphs), nf, ef, out)
+        m.wait()
+        for w, (_, _, out) in zip(want, pins):
+            assert np.array_equal(out.numpy(), w)
+    dev = torch.device("cuda", 0)
+    b = batches[0]
+    with pytest.raises(occu.OccuError):
+        m.predict_async(occu.pack(b.graphs), torch.from_numpy(b.node_feat).to(dev),
+                        torch.from_numpy(b.edge_feat).to(dev), torch.empty(b.num_graphs, device=dev))
