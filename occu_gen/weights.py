@@ -3,16 +3,21 @@
 Layout (SURVEY §8(b) "Weights file"; shapes from P141-P149 read as in
 DESIGN.md R1-R6): for each ANEE layer i = 1..L
     W_u[d][d_in]  W_e[d][d_e_in]  W_m[d][d]  a_s[d]  a_d[d]
-with d_in = F_n, d_e_in = F_e for i = 1 and d otherwise; then the MLP head
-(P125)  W_1[d_h][d]  b_1[d_h]  w_2[d_h]  b_2[1].
+with d_in = F_n, d_e_in = F_e for i = 1 and d otherwise; with the Set-Transformer
+decoder readout (readout = 1, R30-R34) the decoder's
+parameters follow (seeds S[k][d]; the pre-pooling FFN P_*; the two MABs M1_*, M2_* each
+Wq bq Wk bk Wv bv Wo bo ln1_g ln1_b F_W1 F_b1 F_W2 F_b2 ln2_g ln2_b; the final FFN D_*);
+then the MLP head (P125)  W_1[d_h][k·d or d]  b_1[d_h]  w_2[d_h]  b_2[1].
 
 Initialisation: element j of the flat parameter vector (file order) is
 float32((2*u_j - 1) * bound(tensor)), u_j = splitmix64 uniform #j for the
-seed, bound = 1/sqrt(fan_in) (PyTorch-Linear-like).  The C
-library's ``occu_init_weights`` implements the same rule independently.
+seed, bound = 1/sqrt(fan_in) (PyTorch-Linear-like); LayerNorm gains are 1 and
+biases 0 (PyTorch's LayerNorm init).  The C library's ``occu_init_weights`` implements the
+same rule independently.
 
-File: b"OCCUW001", u32[8] = (version=1, L, F_n, F_e, d, d_h, aggr, msg),
-f32 slope, f32 payload (flat, file order), u64 FNV-1a of the payload bytes.
+File: b"OCCUW001", u32[8] = (version, L, F_n, F_e, d, d_h, aggr, msg), f32 slope,
+[version 2 only: u32[3] = (readout, k, heads)], f32 payload (flat, file order), u64
+FNV-1a of the payload bytes.  Version 1 = mean readout, version 2 = decoder readout.
 No method arithmetic lives here.
 """
 from __future__ import annotations
@@ -41,6 +46,9 @@ class ModelConfig:
     aggr: int = AGGR_SUM
     msg: int = MSG_CHANNEL_SOFTMAX
     slope: float = 0.01
+    readout: int = 0        # 0: segmented mean (a7), 1: Set-Transformer decoder (NEXT-2)
+    k: int = 4              # decoder seeds
+    heads: int = 4          # decoder attention heads
 
 
 def param_specs(cfg: ModelConfig):
@@ -56,9 +64,22 @@ def param_specs(cfg: ModelConfig):
             (f"a_s{i}", (cfg.d,), 2 * cfg.d),
             (f"a_d{i}", (cfg.d,), 2 * cfg.d),
         ]
+    d = cfg.d
+    hin = d
+    if cfg.readout == 1:
+        # fan_in -1: constant 1 (LayerNorm gain), 0: constant 0 (LayerNorm bias)
+        lin = lambda p: [(f"{p}W1", (d, d), d), (f"{p}b1", (d,), d), (f"{p}W2", (d, d), d), (f"{p}b2", (d,), d)]
+        specs += [("S", (cfg.k, d), d)] + lin("P_")
+        for m in ("M1_", "M2_"):
+            for w in ("q", "k", "v", "o"):
+                specs += [(f"{m}W{w}", (d, d), d), (f"{m}b{w}", (d,), d)]
+            specs += [(f"{m}ln1_g", (d,), -1), (f"{m}ln1_b", (d,), 0)] + lin(f"{m}F_")
+            specs += [(f"{m}ln2_g", (d,), -1), (f"{m}ln2_b", (d,), 0)]
+        specs += lin("D_")
+        hin = cfg.k * d
     specs += [
-        ("W_1", (cfg.d_h, cfg.d), cfg.d),
-        ("b_1", (cfg.d_h,), cfg.d),
+        ("W_1", (cfg.d_h, hin), hin),
+        ("b_1", (cfg.d_h,), hin),
         ("w_2", (cfg.d_h,), cfg.d_h),
         ("b_2", (1,), cfg.d_h),
     ]
@@ -76,9 +97,12 @@ def init_flat(cfg: ModelConfig, seed: int) -> np.ndarray:
     off = 0
     for _, shape, fan_in in specs:
         n = int(np.prod(shape))
-        u = uniform01(seed, n, off)
-        bound = 1.0 / math.sqrt(float(fan_in))
-        out[off:off + n] = ((2.0 * u - 1.0) * bound).astype(np.float32)
+        if fan_in <= 0:
+            out[off:off + n] = 1.0 if fan_in < 0 else 0.0
+        else:
+            u = uniform01(seed, n, off)
+            bound = 1.0 / math.sqrt(float(fan_in))
+            out[off:off + n] = ((2.0 * u - 1.0) * bound).astype(np.float32)
         off += n
     return out
 
@@ -114,9 +138,11 @@ def write_weights(path: str, cfg: ModelConfig, flat: np.ndarray) -> None:
     payload = flat.tobytes()
     with open(path, "wb") as f:
         f.write(MAGIC)
-        f.write(struct.pack("<8I", VERSION, cfg.L, cfg.F_n, cfg.F_e, cfg.d, cfg.d_h,
-                            cfg.aggr, cfg.msg))
+        f.write(struct.pack("<8I", 2 if cfg.readout else VERSION, cfg.L, cfg.F_n, cfg.F_e, cfg.d,
+                            cfg.d_h, cfg.aggr, cfg.msg))
         f.write(struct.pack("<f", cfg.slope))
+        if cfg.readout:
+            f.write(struct.pack("<3I", cfg.readout, cfg.k, cfg.heads))
         f.write(payload)
         f.write(struct.pack("<Q", fnv1a64(payload)))
 

@@ -85,7 +85,11 @@ def read_weights(path):
     version, L, F_n, F_e, d, d_h, aggr, msg = struct.unpack_from("<8I", raw, 8)
     (slope,) = struct.unpack_from("<f", raw, 40)
     cfg = dict(L=L, F_n=F_n, F_e=F_e, d=d, d_h=d_h, aggr=aggr, msg=msg, slope=float(slope))
-    flat = np.frombuffer(raw, dtype="<f4", offset=44, count=(len(raw) - 52) // 4)
+    hdr = 44
+    if version == 2:                      # Set-Transformer decoder readout (NEXT-2)
+        cfg["readout"], cfg["k"], cfg["heads"] = struct.unpack_from("<3I", raw, 44)
+        hdr = 56
+    flat = np.frombuffer(raw, dtype="<f4", offset=hdr, count=(len(raw) - hdr - 8) // 4)
     return cfg, unflatten(cfg, flat.astype(np.float64))
 
 
@@ -98,7 +102,20 @@ def param_shapes(cfg):
         out += [(f"W_u{i}", (cfg["d"], d_in)), (f"W_e{i}", (cfg["d"], de_in)),
                 (f"W_m{i}", (cfg["d"], cfg["d"])), (f"a_s{i}", (cfg["d"],)),
                 (f"a_d{i}", (cfg["d"],))]
-    out += [("W_1", (cfg["d_h"], cfg["d"])), ("b_1", (cfg["d_h"],)),
+    d, hin = cfg["d"], cfg["d"]
+    if cfg.get("readout", 0) == 1:
+        # Set-Transformer decoder (P159-P205; R30-R34): seeds, pre-pooling FFN,
+        # MAB1 (PMA), MAB2 (SAB), final FFN; the head then reads the flattened k x d output
+        ffn = lambda p: [(p + "W1", (d, d)), (p + "b1", (d,)), (p + "W2", (d, d)), (p + "b2", (d,))]
+        out += [("S", (cfg["k"], d))] + ffn("P_")
+        for m in ("M1_", "M2_"):
+            for w in "qkvo":
+                out += [(m + "W" + w, (d, d)), (m + "b" + w, (d,))]
+            out += [(m + "ln1_g", (d,)), (m + "ln1_b", (d,))] + ffn(m + "F_")
+            out += [(m + "ln2_g", (d,)), (m + "ln2_b", (d,))]
+        out += ffn("D_")
+        hin = cfg["k"] * d
+    out += [("W_1", (cfg["d_h"], hin)), ("b_1", (cfg["d_h"],)),
             ("w_2", (cfg["d_h"],)), ("b_2", (1,))]
     return out
 
@@ -197,9 +214,9 @@ def anee_layer(params, i, cfg, pk, h_prev, e_prev):
     return dict(P=P, hbar=hbar, p=p, q=q, alpha=alpha, z=z, e=e, v=v, g=g, A=A, h=h)
 
 
-def forward(params, cfg, pk, node_feat, edge_feat):
-    """Full forward.  node_feat [N,F_n] in graph-concatenated order; edge_feat
-    [E,F_e] in INPUT edge order (permuted to in-CSR order here, step a1)."""
+def forward_anee(params, cfg, pk, node_feat, edge_feat):
+    """Full forward with the mean readout.  node_feat [N,F_n] in graph-concatenated order;
+    edge_feat [E,F_e] in INPUT edge order (permuted to in-CSR order here, step a1)."""
     h = np.asarray(node_feat, np.float64)
     e = np.asarray(edge_feat, np.float64)[pk["in_eid"].astype(np.int64)]
     layers = []
@@ -207,6 +224,10 @@ def forward(params, cfg, pk, node_feat, edge_feat):
         lay = anee_layer(params, i, cfg, pk, h, e)
         layers.append(lay)
         h, e = lay["h"], lay["e"]
+    out = dict(layers=layers, e0=np.asarray(edge_feat, np.float64)[pk["in_eid"].astype(np.int64)],
+               h0=np.asarray(node_feat, np.float64))
+    if cfg.get("readout", 0) == 1:         # the decoder readout follows in forward()
+        return out
     n_b = np.diff(pk["node_off"].astype(np.int64))
     # north_star: segmented per-graph readout, mean over nodes (R11)
     r = segment_sum(h, pk["node_graph"].astype(np.int64), pk["num_graphs"]) / n_b[:, None]
@@ -214,8 +235,8 @@ def forward(params, cfg, pk, node_feat, edge_feat):
     c = r @ params["W_1"].T + params["b_1"]
     o = leaky_relu(c, cfg["slope"])
     yhat = o @ params["w_2"] + params["b_2"][0]
-    return dict(layers=layers, e0=np.asarray(edge_feat, np.float64)[pk["in_eid"].astype(np.int64)],
-                h0=np.asarray(node_feat, np.float64), r=r, c=c, o=o, yhat=yhat)
+    out.update(r=r, c=c, o=o, yhat=yhat)
+    return out
 
 
 # --------------------------------------------------------------------------
@@ -277,6 +298,70 @@ def forward_bf16(params, cfg, pk, node_feat, edge_feat, rnd=None):
                 r=r, c=c, o=o, yhat=yhat)
 
 
+# --------------------------------------------------------------------------
+# NEXT-2: Set-Transformer decoder readout (P159-P205; R30-R34).
+#   MAB(X, Y) = LN(H̄ + FFN(H̄)),  H̄ = LN(X + MHA(X, Y, Y))          P159-P161, P191-P193
+#   SAB(X) = MAB(X, X)                                               P195-P197
+#   PMA_k(H) = MAB(S, FFN(H)),  S ∈ ℝ^{k×d} learnable seeds           P199-P201
+#   Decoder(H) = FFN(SAB(PMA_k(H))) ∈ ℝ^{k×d}                         P203-P205
+# FFN(x) = W2·ReLU(W1 x + b1) + b2 (R31); MHA with `heads` heads of width d/heads, scaled
+# dot-product attention, input / output projections with biases (R32); LN = LayerNorm with
+# gain and bias, eps 1e-5, biased variance (R33).  The head reads the flattened k·d output.
+# --------------------------------------------------------------------------
+def layer_norm(x, g, b, eps=1e-5):
+    mu = x.mean(axis=-1, keepdims=True)
+    var = ((x - mu) ** 2).mean(axis=-1, keepdims=True)
+    return (x - mu) / np.sqrt(var + eps) * g + b
+
+
+def ffn(x, params, p):
+    return np.maximum(x @ params[p + "W1"].T + params[p + "b1"], 0.0) @ params[p + "W2"].T + params[p + "b2"]
+
+
+def mha(X, Y, params, m, heads):
+    """Multi-head attention MHA(X, Y, Y): queries from X, keys and values from Y."""
+    Q = X @ params[m + "Wq"].T + params[m + "bq"]
+    K = Y @ params[m + "Wk"].T + params[m + "bk"]
+    V = Y @ params[m + "Wv"].T + params[m + "bv"]
+    dh = Q.shape[1] // heads
+    out = np.zeros_like(Q)
+    for h in range(heads):
+        sl = slice(h * dh, (h + 1) * dh)
+        A = softmax_channels(Q[:, sl] @ K[:, sl].T / np.sqrt(dh))     # softmax over the keys
+        out[:, sl] = A @ V[:, sl]
+    return out @ params[m + "Wo"].T + params[m + "bo"]
+
+
+def mab(X, Y, params, m, heads):
+    Hb = layer_norm(X + mha(X, Y, params, m, heads), params[m + "ln1_g"], params[m + "ln1_b"])
+    return layer_norm(Hb + ffn(Hb, params, m + "F_"), params[m + "ln2_g"], params[m + "ln2_b"])
+
+
+def set_decoder(H, params, heads):
+    """Decoder(H) for one graph's node states H [n, d] -> [k, d]."""
+    Z = ffn(H, params, "P_")                           # PMA's FFN(H)
+    pma = mab(params["S"], Z, params, "M1_", heads)    # PMA_k
+    sab = mab(pma, pma, params, "M2_", heads)          # SAB
+    return ffn(sab, params, "D_")
+
+
+def forward(params, cfg, pk, node_feat, edge_feat):
+    """forward_anee + readout: the segmented mean (a7) or, with cfg["readout"] == 1, the
+    Set-Transformer decoder per graph (NEXT-2), then the MLP head on its flattened output."""
+    f = forward_anee(params, cfg, pk, node_feat, edge_feat)
+    if cfg.get("readout", 0) != 1:
+        return f
+    hL = f["layers"][-1]["h"]
+    off = pk["node_off"].astype(np.int64)
+    D = np.stack([set_decoder(hL[off[b]:off[b + 1]], params, cfg["heads"])
+                  for b in range(pk["num_graphs"])])
+    r = D.reshape(pk["num_graphs"], -1)
+    c = r @ params["W_1"].T + params["b_1"]
+    o = leaky_relu(c, cfg["slope"])
+    f.update(dec=D, r=r, c=c, o=o, yhat=o @ params["w_2"] + params["b_2"][0])
+    return f
+
+
 def predict(params, cfg, graphs, node_feat, edge_feat):
     return forward(params, cfg, pack(graphs), node_feat, edge_feat)["yhat"]
 
@@ -295,6 +380,8 @@ def mse_loss(yhat, y, global_batch=None):
 def backward(params, cfg, pk, fwd, y, global_batch=None, dsig=None):
     """dsig(layer dict) -> σ'(y) per edge and channel; default e'(1 - e') (exact
     derivative of σ at y = α z).  backward_bf16 passes e'·σ(-α z) (R28)."""
+    if cfg.get("readout", 0) == 1:
+        raise NotImplementedError("training with the decoder readout (NEXT-2) is inference-only here")
     slope = cfg["slope"]
     B = pk["num_graphs"]
     nb = B if global_batch is None else global_batch

@@ -524,3 +524,124 @@ def test_backward_bf16_within_the_bf16_budget():
     assert abs(lb - la) <= 2e-2 * la
     for k in p:
         assert np.linalg.norm(gb[k] - ga[k]) <= 3e-2 * np.linalg.norm(ga[k]), k
+
+
+# ------------------------------------------ NEXT-2: Set-Transformer decoder readout
+def dec_cfg(k=4, heads=4, d=16, L=2):
+    c = cfg_dict(L=L, F_n=80, F_e=4, d=d, d_h=8)
+    c.update(readout=1, k=k, heads=heads)
+    return c
+
+
+def dec_params(c, seed):
+    wc = weights.ModelConfig(L=c["L"], F_n=c["F_n"], F_e=c["F_e"], d=c["d"], d_h=c["d_h"],
+                             readout=1, k=c["k"], heads=c["heads"])
+    p = oracle.unflatten(c, weights.init_flat(wc, seed).astype(np.float64))
+    for i in range(c["L"]):
+        p[f"W_u{i}"] *= 4.0                      # keep node states O(1) through the layers
+    rng = np.random.default_rng(seed)
+    for m in ("M1_", "M2_"):                      # non-trivial LayerNorm affine parameters
+        for ln in ("ln1", "ln2"):
+            p[m + ln + "_g"] = 1.0 + 0.3 * rng.standard_normal(c["d"])
+            p[m + ln + "_b"] = 0.2 * rng.standard_normal(c["d"])
+    return p
+
+
+def torch_decoder(H, p, c):
+    """Independent implementation of Decoder(H) = FFN(SAB(PMA_k(FFN(H)))) with torch's own
+    nn.MultiheadAttention and nn.LayerNorm (float64)."""
+    torch = pytest.importorskip("torch")
+    d, heads = c["d"], c["heads"]
+    T = lambda a: torch.tensor(a, dtype=torch.float64)
+    F = torch.nn.functional
+
+    def ffn(x, q):
+        return F.linear(F.relu(F.linear(x, T(p[q + "W1"]), T(p[q + "b1"]))), T(p[q + "W2"]), T(p[q + "b2"]))
+
+    def mab(X, Y, m):
+        att = torch.nn.MultiheadAttention(d, heads, bias=True, batch_first=True, dtype=torch.float64)
+        ln1 = torch.nn.LayerNorm(d, eps=1e-5, dtype=torch.float64)
+        ln2 = torch.nn.LayerNorm(d, eps=1e-5, dtype=torch.float64)
+        with torch.no_grad():
+            att.in_proj_weight.copy_(torch.cat([T(p[m + "Wq"]), T(p[m + "Wk"]), T(p[m + "Wv"])]))
+            att.in_proj_bias.copy_(torch.cat([T(p[m + "bq"]), T(p[m + "bk"]), T(p[m + "bv"])]))
+            att.out_proj.weight.copy_(T(p[m + "Wo"]))
+            att.out_proj.bias.copy_(T(p[m + "bo"]))
+            ln1.weight.copy_(T(p[m + "ln1_g"])); ln1.bias.copy_(T(p[m + "ln1_b"]))
+            ln2.weight.copy_(T(p[m + "ln2_g"])); ln2.bias.copy_(T(p[m + "ln2_b"]))
+            a, _ = att(X[None], Y[None], Y[None], need_weights=False)
+            Hb = ln1(X + a[0])
+            return ln2(Hb + ffn(Hb, m + "F_"))
+
+    with torch.no_grad():
+        Z = ffn(T(H), "P_")
+        pma = mab(T(p["S"]), Z, "M1_")
+        return ffn(mab(pma, pma, "M2_"), "D_").numpy()
+
+
+@pytest.mark.parametrize("k,heads", [(4, 4), (1, 2), (3, 1)])
+def test_decoder_matches_torch_modules(k, heads):
+    c = dec_cfg(k=k, heads=heads)
+    b = configs.random_dag_batch(4, 77 + k, max_nodes=20, hub=True)
+    p = dec_params(c, 5 + k)
+    pk = oracle.pack(b.graphs)
+    f = oracle.forward(p, c, pk, b.node_feat, b.edge_feat)
+    hL = f["layers"][-1]["h"]
+    off = pk["node_off"]
+    for g in range(pk["num_graphs"]):
+        ref = torch_decoder(hL[off[g]:off[g + 1]], p, c)
+        assert f["dec"][g].shape == (k, c["d"])
+        assert np.allclose(f["dec"][g], ref, rtol=1e-10, atol=1e-12), g
+    # the head reads the flattened decoder output
+    r = f["dec"].reshape(pk["num_graphs"], -1)
+    y = oracle.leaky_relu(r @ p["W_1"].T + p["b_1"], c["slope"]) @ p["w_2"] + p["b_2"][0]
+    assert np.array_equal(y, f["yhat"])
+
+
+def test_decoder_single_key_attention_ignores_query_and_key_maps():
+    """Softmax over one key is exactly 1: with k = 1 the SAB's attention output is its value
+    projection, so W_q, W_k of MAB2 cannot matter (bitwise); with single-node graphs the same
+    holds for MAB1 (PMA)."""
+    c = dec_cfg(k=1, heads=2)
+    b = configs.random_dag_batch(3, 41, max_nodes=12)
+    p = dec_params(c, 9)
+    pk = oracle.pack(b.graphs)
+    y0 = oracle.forward(p, c, pk, b.node_feat, b.edge_feat)["yhat"]
+    q = dict(p)
+    q["M2_Wq"] = p["M2_Wq"] * 3.0 + 1.0
+    q["M2_Wk"] = -p["M2_Wk"]
+    q["M2_bq"] = p["M2_bq"] + 2.0
+    assert np.array_equal(oracle.forward(q, c, pk, b.node_feat, b.edge_feat)["yhat"], y0)
+    single = [(1, np.zeros(0, np.int32), np.zeros(0, np.int32))] * 3
+    nf = np.random.default_rng(2).normal(size=(3, 80))
+    ef = np.zeros((0, 4))
+    pk1 = oracle.pack(single)
+    y1 = oracle.forward(p, c, pk1, nf, ef)["yhat"]
+    q = dict(p)
+    q["M1_Wq"] = p["M1_Wq"] * 2.0
+    q["M1_Wk"] = p["M1_Wk"] - 1.0
+    assert np.array_equal(oracle.forward(q, c, pk1, nf, ef)["yhat"], y1)
+
+
+def test_decoder_readout_node_permutation_and_batching_invariance():
+    c = dec_cfg()
+    b = configs.random_dag_batch(5, 123, max_nodes=25, hub=True)
+    p = dec_params(c, 3)
+    y = oracle.predict(p, c, b.graphs, b.node_feat, b.edge_feat)
+    for g in range(b.num_graphs):                       # batching (BLAS blocking: ~1 ulp)
+        s = b.subset([g])
+        assert np.allclose(oracle.predict(p, c, s.graphs, s.node_feat, s.edge_feat), y[g:g + 1],
+                           rtol=1e-13, atol=1e-15)
+    # relabel nodes inside every graph: PMA pools a set, so ŷ is unchanged up to rounding
+    rng = np.random.default_rng(8)
+    graphs, nfs, efs = [], [], []
+    noff = np.concatenate([[0], np.cumsum([g[0] for g in b.graphs])])
+    eoff = np.concatenate([[0], np.cumsum([len(g[1]) for g in b.graphs])])
+    for g, (n, s_, t_) in enumerate(b.graphs):
+        perm = rng.permutation(n)
+        inv = np.argsort(perm)
+        graphs.append((n, inv[s_].astype(np.int32), inv[t_].astype(np.int32)))
+        nfs.append(b.node_feat[noff[g]:noff[g + 1]][perm])
+        efs.append(b.edge_feat[eoff[g]:eoff[g + 1]])
+    y2 = oracle.predict(p, c, graphs, np.concatenate(nfs), np.concatenate(efs))
+    assert np.allclose(y2, y, rtol=1e-12, atol=1e-14)
