@@ -453,6 +453,33 @@ def main():
                     "what": "ANEE reading B: per-channel softmax over each destination's in-edges"}
         del mr
 
+    # ---- NEXT-2: Set-Transformer decoder readout (k = 4 seeds, 4 heads), inference, same batch
+    decoder = None
+    if not args.no_bf16 and args.path == 0:
+        md = occu.Model(occu.config(L=3, F_n=80, F_e=4, d=128, readout=occu.READOUT_SET_DECODER,
+                                    k=4, heads=4), device=local, stream=stream.cuda_stream)
+        md.init_weights(42)
+        outd = torch.empty_like(out)
+        inferd = lambda: md.predict(csr, nf, ef, outd)
+        timed(inferd, args.warmup, mdl=md)
+        bar()
+        td_, ld_ = timed(inferd, args.steps, mdl=md)
+        bar()
+        timed(inferd, args.steps, profile=True, mdl=md)
+        bar()
+        msd = max_over_ranks(float(np.sum(td_)) / args.steps)
+        algd = algorithmic_bytes(N, E, B, d)                  # h_L stored: unfused gather
+        algd["dec_ffn_tc"] = 2 * (4 * N * d + 4 * N * d)       # T = FFN1(h_L), Z = FFN2(T)
+        algd["set_decoder"] = 4 * N * d + 4 * (B + 1) + 4 * B * (4 * d + 130)
+        kd, roofd = kernel_table(md.profile(), algd, {})
+        decoder = {"value": B * world / (msd * 1e-3), "unit": "graphs/s", "ms_per_step": msd,
+                   "dtype": "f32", "gpu_launches": ld_, "roofline": roofd,
+                   "kernel_ms_per_step": {k_: v["ms_per_step"] for k_, v in kd.items()},
+                   "kernels": kd,
+                   "what": "readout = Set-Transformer decoder FFN(SAB(PMA_4(FFN(h_L)))), 4 heads, "
+                           "head on the flattened 4 x 128 output (P159-P205)"}
+        del md
+
     # ---- e2e through the public API with host buffers (pinned), pack included
     pin_nf = torch.from_numpy(batch.node_feat).pin_memory()
     pin_ef = torch.from_numpy(batch.edge_feat).pin_memory()
@@ -585,6 +612,7 @@ def main():
             "e2e": e2e,
             "bf16": bf16,
             "readingb": readingb,
+            "decoder": decoder,
             "train": train,
             "cpu_baseline": cpu,
         }

@@ -57,17 +57,24 @@ typedef enum { OCCU_AGGR_SUM = 0, OCCU_AGGR_MEAN = 1 } occu_aggr;            /* 
 typedef enum { OCCU_MSG_CHANNEL_SOFTMAX = 0, OCCU_MSG_NEIGHBOR_SOFTMAX = 1 } occu_msg; /* R4 */
 typedef enum { OCCU_FP32 = 0, OCCU_BF16 = 1 } occu_precision;
 
-/* Model configuration.  L ANEE rounds of width d; raw feature widths F_n
- * (node, Table I) and F_e (edge); head hidden width d_h; LeakyReLU slope
- * (R7, 0.01).  d must be a multiple of 32 and <= 256 (kernel tiling);
- * F_n, F_e multiples of 4.  msg = OCCU_MSG_NEIGHBOR_SOFTMAX is reserved
- * (NEXT-1) and rejected with OCCU_EINVAL by this build. */
+typedef enum { OCCU_READOUT_MEAN = 0, OCCU_READOUT_SET_DECODER = 1 } occu_readout;
+
+/* Model configuration.  L ANEE rounds of width d (64 or 128 in this build); raw feature
+ * widths F_n (node, Table I) and F_e (edge); head hidden width d_h; LeakyReLU slope (R7,
+ * 0.01); F_n, F_e multiples of 4.  msg = OCCU_MSG_NEIGHBOR_SOFTMAX (reading B, NEXT-1):
+ * OCCU_FP32, kernel path 0.  readout: OCCU_READOUT_MEAN (a7, the north_star's segmented
+ * mean; default when the trailing fields are zero) or OCCU_READOUT_SET_DECODER (P159-P205,
+ * NEXT-2: Decoder(H) = FFN(SAB(PMA_k(H))) per graph, k seeds, `heads` attention heads, the
+ * head reading the flattened k·d output; OCCU_FP32, kernel path 0, inference only: training
+ * returns OCCU_EINVAL); k in [1, 8], heads in {1, 2, 4, 8}, k·heads <= 16. */
 typedef struct {
   int32_t L, F_n, F_e, d, d_h;
   int32_t aggr;      /* occu_aggr */
   int32_t msg;       /* occu_msg */
   int32_t prec;      /* occu_precision */
   float slope;
+  int32_t readout;   /* occu_readout */
+  int32_t k, heads;  /* decoder seeds and heads (readout = OCCU_READOUT_SET_DECODER) */
 } occu_config;
 
 /* One caller-owned input graph (host memory), local node ids. */
@@ -179,7 +186,7 @@ typedef enum {
   OCCU_T_Q = 2,      /* [N]     layer l */
   OCCU_T_E = 3,      /* [E][d]  layer l, in-CSR edge order */
   OCCU_T_H = 4,      /* [N][d]  layer l */
-  OCCU_T_R = 5,      /* [B][d]  readout */
+  OCCU_T_R = 5,      /* [B][d]  readout ([B][k·d] flattened decoder output with the decoder) */
   OCCU_T_YHAT = 6    /* [B] */
 } occu_tensor;
 /* Kernel path: 0 (default) = tcgen05 tensor cores (fp16x2-split GEMMs with

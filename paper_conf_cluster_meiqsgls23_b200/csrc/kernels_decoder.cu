@@ -1,0 +1,392 @@
+// NEXT-2 readout: the Set-Transformer decoder of P159-P205 (R30-R34),
+//   Decoder(H) = FFN(SAB(PMA_k(H))),  PMA_k(H) = MAB(S, FFN(H)),  SAB(X) = MAB(X, X),
+//   MAB(X, Y) = LN(H̄ + FFN(H̄)),  H̄ = LN(X + MHA(X, Y, Y)),
+// per graph over its last-layer node states, then the MLP head on the flattened k·d output.
+//
+// B200 mapping:
+//  * FFN(H) over all N nodes is the only large contraction: two tensor-core row-GEMMs with a
+//    bias (+ReLU) epilogue (launch_bias_tc), T = ReLU(h W1ᵀ + b1), Z = T W2ᵀ + b2.
+//  * MHA(S, Z, Z) needs no per-node key / value projections: the score of node n for seed j
+//    in head h is (Q_j,h · (W_k Z_n + b_k)_h)/√d_h = Z_n · M[:, (j,h)] + c_(j,h) with
+//    M = W_k,hᵀ Q_j,h / √d_h (d x k·heads, built per CTA from the seeds), and since the
+//    attention weights of a (j,h) sum to 1, Σ_n α (W_v Z_n + b_v) = W_v (Σ_n α Z_n) + b_v.  So
+//    the pool streams Z once per graph (32-row chunks staged in shared memory) with an online
+//    softmax per (j,h), accumulating P_(j,h) = Σ_n α Z_n; W_v is applied to the k·heads pooled
+//    vectors only.  Fixed order everywhere (deterministic).
+//  * The rest (W_v, W_o, LayerNorms, the k-element SAB, the FFNs, the head) is k-vector work
+//    per graph: warp-per-output-row GEMVs against L2-resident weights, one CTA per graph.
+#include <cuda_runtime.h>
+#include <math.h>
+#include <stdint.h>
+
+#include "occu_internal.h"
+
+namespace occu {
+namespace {
+
+constexpr int DT = 256;          // threads per CTA
+constexpr int NW = DT / 32;
+constexpr int CH = 32;           // node rows per pooling chunk
+constexpr int KMAX = 8;          // seeds
+constexpr int KHMAX = 16;        // seeds x heads
+constexpr float L2E = 1.4426950408889634f;
+
+struct DecArgs {
+  const float *Z;                // [N][D] FFN(h_L)
+  const int32_t *node_off;       // [B+1]
+  const float *P;                // flat parameters
+  DecLayout L;
+  size_t W_1, b_1, w_2, b_2;
+  int k, heads, d_h;
+  float slope;
+  float *r, *c, *yhat;           // [B][k·D], [B][d_h], [B]
+};
+
+__device__ __forceinline__ float ex2(float x) {
+  float r;
+  asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(r) : "f"(x));
+  return r;
+}
+
+// Y[v·ldy + n] = act(bias[n] + Σ_c W[n·ldw + c] X[v·ldx + c]) for rows n < nrows, vectors
+// v < nvec; warp per row (strided), lanes stride the columns (coalesced row reads), fixed
+// butterfly reduction.  ncols % 4 == 0.
+// Rows are taken RB at a time per warp with all RB row loads issued before use (one L2
+// latency per batch instead of one per row).
+__device__ void warp_gemv(const float *__restrict__ W, int ldw, int ncols, int nrows,
+                          const float *X, int ldx, int nvec, float *Y, int ldy,
+                          const float *__restrict__ bias, bool relu) {
+  constexpr int RB = 8;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  for (int n0 = warp * RB; n0 < nrows; n0 += NW * RB) {
+    for (int c0 = 0; c0 < ncols; c0 += 128) {
+      const int c = c0 + lane * 4;
+      float4 w[RB];
+#pragma unroll
+      for (int q = 0; q < RB; ++q) {
+        const int n = min(n0 + q, nrows - 1);
+        w[q] = c < ncols ? __ldg(reinterpret_cast<const float4 *>(W + long(n) * ldw + c))
+                         : make_float4(0.f, 0.f, 0.f, 0.f);
+      }
+      for (int v = 0; v < nvec; ++v) {
+        float4 x = make_float4(0.f, 0.f, 0.f, 0.f);
+        if (c < ncols) x = *reinterpret_cast<const float4 *>(X + v * ldx + c);
+#pragma unroll
+        for (int q = 0; q < RB; ++q) {
+          float a = w[q].x * x.x + w[q].y * x.y + w[q].z * x.z + w[q].w * x.w;
+#pragma unroll
+          for (int o = 16; o > 0; o >>= 1) a += __shfl_xor_sync(0xffffffffu, a, o);
+          if (lane == 0 && n0 + q < nrows) {
+            float *y = Y + v * ldy + n0 + q;
+            *y = (c0 == 0 ? 0.f : *y) + a;
+          }
+        }
+      }
+    }
+    __syncwarp();
+    if (lane < RB && n0 + lane < nrows)
+      for (int v = 0; v < nvec; ++v) {
+        float *y = Y + v * ldy + n0 + lane;
+        const float a = *y + (bias ? __ldg(bias + n0 + lane) : 0.f);
+        *y = relu ? fmaxf(a, 0.f) : a;
+      }
+    __syncwarp();
+  }
+}
+
+// Y[v] = LN(A[v] + Bv[v]) · g + b over D channels (eps 1e-5, biased variance); warp per vector.
+template <int D>
+__device__ void warp_add_ln(const float *A, const float *Bv, float *Y, int nvec,
+                            const float *__restrict__ g, const float *__restrict__ b) {
+  constexpr int V = D / 32;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  for (int v = warp; v < nvec; v += NW) {
+    float x[V], s = 0.f;
+#pragma unroll
+    for (int i = 0; i < V; ++i) {
+      x[i] = A[v * D + lane + 32 * i] + Bv[v * D + lane + 32 * i];
+      s += x[i];
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+    const float mu = s / float(D);
+    float q = 0.f;
+#pragma unroll
+    for (int i = 0; i < V; ++i) q = fmaf(x[i] - mu, x[i] - mu, q);
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) q += __shfl_xor_sync(0xffffffffu, q, o);
+    const float inv = rsqrtf(q / float(D) + 1e-5f);
+#pragma unroll
+    for (int i = 0; i < V; ++i) {
+      const int ch = lane + 32 * i;
+      Y[v * D + ch] = (x[i] - mu) * inv * __ldg(g + ch) + __ldg(b + ch);
+    }
+  }
+}
+
+// Once per forward (one CTA): PMA queries Q = S W_qᵀ + b_q, the folded key map
+// M[c][(j,h)] = Σ_i Q[j][h·dh+i] W_k[h·dh+i][c] / √dh and c_(j,h) = Q_j,h · b_k,h / √dh.
+template <int D>
+__global__ void __launch_bounds__(DT) set_decoder_prep_kernel(const DecArgs a, float *__restrict__ prep) {
+  __shared__ __align__(16) float S[KMAX * D], Q[KMAX * D];
+  const int k = a.k, heads = a.heads, KH = k * heads, dh = D / heads, t = threadIdx.x;
+  const float *P = a.P;
+  const DecLayout &L = a.L;
+  pdl_trigger();
+  pdl_wait();
+  for (int i = t; i < k * D; i += DT) S[i] = P[L.S + i];
+  __syncthreads();
+  warp_gemv(P + L.M1.Wq, D, D, D, S, D, k, Q, D, P + L.M1.bq, false);
+  __syncthreads();
+  const float isq = rsqrtf(float(dh));
+  for (int o = t; o < D * KH; o += DT) {
+    const int c = o % D, kh = o / D, j = kh / heads, h = kh % heads;
+    float m0 = 0.f, m1 = 0.f, m2 = 0.f, m3 = 0.f;
+    for (int i = 0; i < dh; i += 4) {
+      m0 = fmaf(Q[j * D + h * dh + i], __ldg(P + L.M1.Wk + long(h * dh + i) * D + c), m0);
+      m1 = fmaf(Q[j * D + h * dh + i + 1], __ldg(P + L.M1.Wk + long(h * dh + i + 1) * D + c), m1);
+      m2 = fmaf(Q[j * D + h * dh + i + 2], __ldg(P + L.M1.Wk + long(h * dh + i + 2) * D + c), m2);
+      m3 = fmaf(Q[j * D + h * dh + i + 3], __ldg(P + L.M1.Wk + long(h * dh + i + 3) * D + c), m3);
+    }
+    prep[c * KHMAX + kh] = ((m0 + m1) + (m2 + m3)) * isq;
+  }
+  if (t < KH) {
+    const int j = t / heads, h = t % heads;
+    float m = 0.f;
+    for (int i = 0; i < dh; ++i) m = fmaf(Q[j * D + h * dh + i], __ldg(P + L.M1.bk + h * dh + i), m);
+    prep[D * KHMAX + t] = m * isq;
+  }
+}
+
+template <int D>
+__global__ void __launch_bounds__(DT) set_decoder_kernel(const DecArgs a, const float *__restrict__ prep) {
+  extern __shared__ __align__(16) float sm[];
+  const int k = a.k, heads = a.heads, KH = k * heads, dh = D / heads;
+  float *Zc = sm;                          // [CH][D]
+  float *sc = Zc + CH * D;                 // [CH][KHMAX]  scores, then weights
+  float *Msm = sc + CH * KHMAX;            // [CH][NW][KHMAX] score partials
+  float *Pacc = Msm + CH * NW * KHMAX;     // [KHMAX][D]
+  float *buf = Pacc + KHMAX * D;           // 6 x [KMAX][D]
+  float *B0 = buf, *B1 = B0 + KMAX * D, *B2 = B1 + KMAX * D, *B3 = B2 + KMAX * D,
+        *B4 = B3 + KMAX * D, *B5 = B4 + KMAX * D;
+  float *cst = B5 + KMAX * D;              // [KHMAX]
+  float *mrun = cst + KHMAX, *lrun = mrun + KHMAX, *scl = lrun + KHMAX;
+  float *cvec = scl + KHMAX;               // [d_h]
+  const int t = threadIdx.x;
+  const float *P = a.P;
+  const DecLayout &L = a.L;
+  const int g = blockIdx.x;
+  const long u0 = a.node_off[g], u1 = a.node_off[g + 1];
+  pdl_trigger();
+  pdl_wait();
+
+  // ---- the folded key map M, c of the seeds' queries (set_decoder_prep_kernel, R32);
+  // thread t keeps M[cg·CPG .. +CPG][t & 15] in registers for the score dots
+  constexpr int CPG = D / 16;              // channels per group (16 groups of the 256 threads)
+  const int cg = t >> 4;
+  float mreg[CPG];
+#pragma unroll
+  for (int i = 0; i < CPG; ++i) mreg[i] = __ldg(prep + (cg * CPG + i) * KHMAX + (t & 15));
+  float *red = Msm;                        // [CH][NW][KHMAX] score partials (M lives in registers)
+  const float isq = rsqrtf(float(dh));
+  if (t < KH) {
+    cst[t] = prep[D * KHMAX + t];
+    mrun[t] = -INFINITY;
+    lrun[t] = 0.f;
+  }
+  for (int i = t; i < KH * D; i += DT) Pacc[i] = 0.f;
+  __syncthreads();
+
+  // ---- attention pool over the graph's nodes: online softmax per (seed, head)
+  for (long n0 = u0; n0 < u1; n0 += CH) {
+    const int rows = int(min(long(CH), u1 - n0));
+    for (int i = t; i < rows * (D / 4); i += DT) {
+      const int r = i / (D / 4), c4 = i % (D / 4);
+      reinterpret_cast<float4 *>(Zc + r * D)[c4] =
+          __ldg(reinterpret_cast<const float4 *>(a.Z + (n0 + r) * D) + c4);
+    }
+    __syncthreads();
+    {   // scores: thread (kh, channel group) holds its M slice in registers; partial dots of
+        // the two channel groups of a warp combined by shuffle, the NW warp partials in smem
+      for (int r = 0; r < rows; ++r) {
+        const float *zr = Zc + r * D + cg * CPG;
+        float part = 0.f;
+#pragma unroll
+        for (int i = 0; i < CPG; i += 4) {
+          const float4 z = *reinterpret_cast<const float4 *>(zr + i);
+          part = fmaf(z.x, mreg[i], fmaf(z.y, mreg[i + 1], fmaf(z.z, mreg[i + 2], fmaf(z.w, mreg[i + 3], part))));
+        }
+        part += __shfl_xor_sync(0xffffffffu, part, 16);
+        if ((t & 16) == 0) red[(r * NW + (t >> 5)) * KHMAX + (t & 15)] = part;
+      }
+      __syncthreads();
+      for (int o = t; o < rows * KH; o += DT) {
+        const int r = o / KH, kh = o % KH;
+        float sacc = cst[kh];
+        for (int w = 0; w < NW; ++w) sacc += red[(r * NW + w) * KHMAX + kh];
+        sc[r * KHMAX + kh] = sacc;
+      }
+    }
+    __syncthreads();
+    {   // warp per (seed, head): lanes = chunk rows; max, weights and their sum by shuffles
+      const int warp = t >> 5, lane = t & 31;
+      for (int kh = warp; kh < KH; kh += NW) {
+        const float sv = lane < rows ? sc[lane * KHMAX + kh] : -INFINITY;
+        float cm = sv;
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) cm = fmaxf(cm, __shfl_xor_sync(0xffffffffu, cm, o));
+        const float mold = mrun[kh];
+        const float mn = fmaxf(mold, cm);
+        const float w = lane < rows ? ex2((sv - mn) * L2E) : 0.f;
+        float ws = w;
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) ws += __shfl_xor_sync(0xffffffffu, ws, o);
+        if (lane < rows) sc[lane * KHMAX + kh] = w;
+        __syncwarp();
+        if (lane == 0) {
+          const float f = ex2((mold - mn) * L2E);               // 0 on the first chunk
+          scl[kh] = f;
+          lrun[kh] = lrun[kh] * f + ws;
+          mrun[kh] = mn;
+        }
+      }
+    }
+    __syncthreads();
+    for (int o4 = t; o4 < KH * D / 4; o4 += DT) {   // 4 consecutive channels of one (j,h)
+      const int kh = o4 / (D / 4), c = (o4 % (D / 4)) * 4;
+      float4 acc = reinterpret_cast<float4 *>(Pacc)[o4];
+      const float f = scl[kh];
+      acc.x *= f; acc.y *= f; acc.z *= f; acc.w *= f;
+      for (int r = 0; r < rows; ++r) {
+        const float w = sc[r * KHMAX + kh];
+        const float4 z = *reinterpret_cast<const float4 *>(Zc + r * D + c);
+        acc.x = fmaf(w, z.x, acc.x); acc.y = fmaf(w, z.y, acc.y);
+        acc.z = fmaf(w, z.z, acc.z); acc.w = fmaf(w, z.w, acc.w);
+      }
+      reinterpret_cast<float4 *>(Pacc)[o4] = acc;
+    }
+    __syncthreads();
+  }
+  for (int o = t; o < KH * D; o += DT) Pacc[o] = Pacc[o] / lrun[o / D];
+  __syncthreads();
+
+  // ---- MAB1 = PMA_k: O = W_v P + b_v per head, X1 = W_o O + b_o, H̄ = LN(S + X1), LN(H̄ + FFN(H̄))
+  for (int h = 0; h < heads; ++h)
+    warp_gemv(P + L.M1.Wv + long(h) * dh * D, D, D, dh, Pacc + h * D, heads * D, k, B0 + h * dh, D,
+              P + L.M1.bv + h * dh, false);
+  __syncthreads();
+  warp_gemv(P + L.M1.Wo, D, D, D, B0, D, k, B1, D, P + L.M1.bo, false);
+  for (int i = t; i < k * D; i += DT) B3[i] = P[L.S + i];
+  __syncthreads();
+  warp_add_ln<D>(B3, B1, B2, k, P + L.M1.ln1_g, P + L.M1.ln1_b);      // B2 = H̄1
+  __syncthreads();
+  warp_gemv(P + L.M1.F.W1, D, D, D, B2, D, k, B3, D, P + L.M1.F.b1, true);
+  __syncthreads();
+  warp_gemv(P + L.M1.F.W2, D, D, D, B3, D, k, B4, D, P + L.M1.F.b2, false);
+  __syncthreads();
+  warp_add_ln<D>(B2, B4, B5, k, P + L.M1.ln2_g, P + L.M1.ln2_b);      // B5 = PMA_k(Z)
+  __syncthreads();
+
+  // ---- MAB2 = SAB over the k vectors
+  warp_gemv(P + L.M2.Wq, D, D, D, B5, D, k, B0, D, P + L.M2.bq, false);
+  warp_gemv(P + L.M2.Wk, D, D, D, B5, D, k, B1, D, P + L.M2.bk, false);
+  warp_gemv(P + L.M2.Wv, D, D, D, B5, D, k, B2, D, P + L.M2.bv, false);
+  __syncthreads();
+  // scores / softmax over the k keys per (head, query); Zc reused as [heads][k][k]
+  for (int o = t; o < heads * k * k; o += DT) {
+    const int h = o / (k * k), j = (o / k) % k, jj = o % k;
+    float s = 0.f;
+    for (int i = 0; i < dh; ++i) s = fmaf(B0[j * D + h * dh + i], B1[jj * D + h * dh + i], s);
+    Zc[o] = s * isq;
+  }
+  __syncthreads();
+  for (int o = t; o < heads * k; o += DT) {
+    float m = -INFINITY, l = 0.f;
+    for (int jj = 0; jj < k; ++jj) m = fmaxf(m, Zc[o * k + jj]);
+    for (int jj = 0; jj < k; ++jj) {
+      const float w = ex2((Zc[o * k + jj] - m) * L2E);
+      Zc[o * k + jj] = w;
+      l += w;
+    }
+    for (int jj = 0; jj < k; ++jj) Zc[o * k + jj] /= l;
+  }
+  __syncthreads();
+  for (int o = t; o < k * D; o += DT) {
+    const int j = o / D, ch = o % D, h = ch / dh;
+    float acc = 0.f;
+    for (int jj = 0; jj < k; ++jj) acc = fmaf(Zc[(h * k + j) * k + jj], B2[jj * D + ch], acc);
+    B3[o] = acc;
+  }
+  __syncthreads();
+  warp_gemv(P + L.M2.Wo, D, D, D, B3, D, k, B4, D, P + L.M2.bo, false);
+  __syncthreads();
+  warp_add_ln<D>(B5, B4, B0, k, P + L.M2.ln1_g, P + L.M2.ln1_b);      // B0 = H̄2
+  __syncthreads();
+  warp_gemv(P + L.M2.F.W1, D, D, D, B0, D, k, B1, D, P + L.M2.F.b1, true);
+  __syncthreads();
+  warp_gemv(P + L.M2.F.W2, D, D, D, B1, D, k, B2, D, P + L.M2.F.b2, false);
+  __syncthreads();
+  warp_add_ln<D>(B0, B2, B3, k, P + L.M2.ln2_g, P + L.M2.ln2_b);      // B3 = SAB(PMA_k(Z))
+  __syncthreads();
+
+  // ---- final FFN -> decoder output [k][D] (flattened into r), then the head
+  warp_gemv(P + L.D.W1, D, D, D, B3, D, k, B4, D, P + L.D.b1, true);
+  __syncthreads();
+  warp_gemv(P + L.D.W2, D, D, D, B4, D, k, B5, D, P + L.D.b2, false);
+  __syncthreads();
+  for (int i = t; i < k * D; i += DT) a.r[long(g) * k * D + i] = B5[i];
+  warp_gemv(P + a.W_1, k * D, k * D, a.d_h, B5, 0, 1, cvec, 0, P + a.b_1, false);
+  __syncthreads();
+  if (t < 32) {        // ŷ = w_2 · LReLU(c) + b_2, fixed-order warp reduction
+    float s = 0.f;
+    for (int i = t; i < a.d_h; i += 32) {
+      const float cv = cvec[i];
+      a.c[long(g) * a.d_h + i] = cv;
+      s = fmaf(__ldg(P + a.w_2 + i), cv > 0.f ? cv : a.slope * cv, s);
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+    if (t == 0) a.yhat[g] = s + __ldg(P + a.b_2);
+  }
+}
+
+}  // namespace
+
+int launch_set_decoder(const occu_ctx *ctx, const DevCsr &csr, const float *hL, float *T, float *Z,
+                       float *r, float *c, float *yhat, cudaStream_t st) {
+  const occu_config &cf = ctx->cfg;
+  const ParamLayout &L = ctx->layout;
+  const float *P = ctx->params.as<float>();
+  if (!L.dec || cf.k > KMAX || cf.k * cf.heads > KHMAX) return -int(cudaErrorInvalidValue);
+  int n = 0, rr;
+  if ((rr = launch_bias_tc(ctx, hL, cf.d, csr.N, 0, cf.L, P + L.D.P.b1, true, T, "dec_ffn_tc", st)) < 0) return rr;
+  n += rr;
+  if ((rr = launch_bias_tc(ctx, T, cf.d, csr.N, 1, cf.L, P + L.D.P.b2, false, Z, "dec_ffn_tc", st)) < 0) return rr;
+  n += rr;
+  DecArgs a{};
+  if (const_cast<occu_ctx *>(ctx)->ws.dprep.ensure(size_t(cf.d * KHMAX + KHMAX) * 4) != cudaSuccess)
+    return -int(cudaErrorMemoryAllocation);
+  float *prep = ctx->ws.dprep.as<float>();
+  a.Z = Z; a.node_off = csr.node_off; a.P = P; a.L = L.D;
+  a.W_1 = L.W_1; a.b_1 = L.b_1; a.w_2 = L.w_2; a.b_2 = L.b_2;
+  a.k = cf.k; a.heads = cf.heads; a.d_h = cf.d_h; a.slope = cf.slope;
+  a.r = r; a.c = c; a.yhat = yhat;
+  const int D = cf.d;
+  const size_t smem = size_t(CH * D + CH * KHMAX + CH * NW * KHMAX + KHMAX * D + 6 * KMAX * D +
+                             4 * KHMAX + cf.d_h) * 4;
+  OCCU_PROF_BEGIN(ctx, "set_decoder", st);
+  if (D == 64) {
+    set_decoder_prep_kernel<64><<<1, DT, 0, st>>>(a, prep);
+    cudaFuncSetAttribute(set_decoder_kernel<64>, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
+    launch_pdl(ctx->pdl & 8, set_decoder_kernel<64>, csr.B, DT, smem, st, a, (const float *)prep);
+  } else {
+    set_decoder_prep_kernel<128><<<1, DT, 0, st>>>(a, prep);
+    cudaFuncSetAttribute(set_decoder_kernel<128>, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
+    launch_pdl(ctx->pdl & 8, set_decoder_kernel<128>, csr.B, DT, smem, st, a, (const float *)prep);
+  }
+  OCCU_PROF_END(ctx);
+  const cudaError_t e = cudaGetLastError();
+  return e == cudaSuccess ? n + 2 : -int(e);
+}
+
+}  // namespace occu

@@ -120,6 +120,8 @@ struct RowGemmArgs {
   const float *dh, *h, *hbar, *e, *de;
   const float *mask_h;     // PLAIN: multiply row by LReLU'(mask_h row) (÷ deg for MEAN) -> dA
   int mask_bf;             // mask_h rows are BF16 (OCCU_BF16 training)
+  const float *bias;       // PLAIN: per-column bias (nullable), then ReLU if relu
+  int relu;
   const int32_t *in_ptr;
   int mean;
   float *dal;              // EDGEBWD: dα [R]
@@ -489,6 +491,13 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
                 o[u + t] *= xv[t] > 0.f ? 1.f : a.slope;
                 if (a.mean) o[u + t] = o[u + t] / dsc;
               }
+            }
+          }
+          if (a.bias) {
+#pragma unroll
+            for (int u = 0; u < 16; ++u) {
+              o[u] += __ldg(a.bias + cb + c0 + u);
+              if (a.relu) o[u] = fmaxf(o[u], 0.f);
             }
           }
           if (a.add && live) {
@@ -1692,9 +1701,10 @@ int tc_prepare_weights(occu_ctx *ctx, cudaStream_t st) {
   if (ctx->wimg_version == ctx->params_version) return 0;
   const occu_config &c = ctx->cfg;
   const ParamLayout &L = ctx->layout;
-  if (ctx->wimg.ensure(size_t(c.L) * 6 * WIMG_MAX) != cudaSuccess ||
-      ctx->wfexp.ensure(size_t(c.L) * 6 * 2 * sizeof(int)) != cudaSuccess ||
-      ctx->wjobs.ensure(size_t(c.L) * 6 * sizeof(WImageJob)) != cudaSuccess)
+  // slots: 6 kinds per ANEE layer, plus "layer" L for the decoder's FFN (kinds 0, 1)
+  if (ctx->wimg.ensure(size_t(c.L + 1) * 6 * WIMG_MAX) != cudaSuccess ||
+      ctx->wfexp.ensure(size_t(c.L + 1) * 6 * 2 * sizeof(int)) != cudaSuccess ||
+      ctx->wjobs.ensure(size_t(c.L + 1) * 6 * sizeof(WImageJob)) != cudaSuccess)
     return -int(cudaErrorMemoryAllocation);
   std::vector<WImageJob> jobs;
   const float *P = ctx->params.as<float>();
@@ -1717,6 +1727,17 @@ int tc_prepare_weights(occu_ctx *ctx, cudaStream_t st) {
     add(2, P + L.W_m[i], c.d, c.d, 0);
     add(3, P + L.W_m[i], c.d, c.d, 1);
     if (i > 0) add(5, P + L.W_u[i], c.d, c.d, 1);
+  }
+  if (L.dec) {      // NEXT-2 decoder: the pre-pooling FFN's two d x d matrices
+    auto addd = [&](int kind, const float *W) {
+      WImageJob j;
+      j.W = W; j.D = c.d; j.K = c.d; j.transW = 0; j.bf16 = 0;
+      j.img = const_cast<uint8_t *>(tc_wimg(ctx, kind, c.L));
+      j.fexp = const_cast<int *>(tc_wfexp(ctx, kind, c.L));
+      jobs.push_back(j);
+    };
+    addd(0, P + L.D.P.W1);
+    addd(1, P + L.D.P.W2);
   }
   // job table: pointers are fixed for the ctx, re-uploaded only with the images
   if (cudaMemcpyAsync(ctx->wjobs.ptr, jobs.data(), jobs.size() * sizeof(WImageJob),
@@ -1915,6 +1936,15 @@ static int plain_impl(const occu_ctx *ctx, const float *A, int K, int R, int wki
   return launch_rowgemm<D, EPI_PLAIN>(ctx, r, name, st);
 }
 template <int D>
+static int bias_impl(const occu_ctx *ctx, const float *A, int K, int R, int wkind, int layer,
+                     const float *bias, bool relu, float *out, const char *name, cudaStream_t st) {
+  RowGemmArgs r{};
+  r.slope = ctx->cfg.slope;
+  r.A = A; r.K = K; r.R = R; r.out = out; r.bias = bias; r.relu = relu ? 1 : 0;
+  r.wimg = tc_wimg(ctx, wkind, layer); r.wfexp = tc_wfexp(ctx, wkind, layer);
+  return launch_rowgemm<D, EPI_PLAIN>(ctx, r, name, st);
+}
+template <int D>
 static int bwd_edge_impl(const occu_ctx *ctx, const DevCsr &csr, int layer, const float *e_in,
                          int Ke, const float *e, const float *de, const float *p, const float *q,
                          float *DZ, float *dal, cudaStream_t st) {
@@ -1939,6 +1969,12 @@ int launch_plain_tc(const occu_ctx *ctx, const float *A, int K, int R, int wkind
   if (R <= 0) return 0;
   return ctx->cfg.d == 64 ? plain_impl<64>(ctx, A, K, R, wkind, layer, add, out, name, st, mask_h, in_ptr, mask_bf)
                           : plain_impl<128>(ctx, A, K, R, wkind, layer, add, out, name, st, mask_h, in_ptr, mask_bf);
+}
+int launch_bias_tc(const occu_ctx *ctx, const float *A, int K, int R, int wkind, int layer,
+                   const float *bias, bool relu, float *out, const char *name, cudaStream_t st) {
+  if (R <= 0) return 0;
+  return ctx->cfg.d == 64 ? bias_impl<64>(ctx, A, K, R, wkind, layer, bias, relu, out, name, st)
+                          : bias_impl<128>(ctx, A, K, R, wkind, layer, bias, relu, out, name, st);
 }
 int launch_bwd_edge_tc(const occu_ctx *ctx, const DevCsr &csr, int layer, const float *e_in, int Ke,
                        const float *e, const float *de, const float *p, const float *q, float *DZ,

@@ -19,11 +19,20 @@ namespace occu {
 void set_global_error(const std::string &msg);
 const char *global_error();
 
+// Set-Transformer decoder parameters (readout = OCCU_READOUT_SET_DECODER), offsets in floats
+// into the flat parameter vector (file order, occu_gen/weights.py).
+struct FfnOff { size_t W1, b1, W2, b2; };
+struct MabOff { size_t Wq, bq, Wk, bk, Wv, bv, Wo, bo, ln1_g, ln1_b; FfnOff F; size_t ln2_g, ln2_b; };
+struct DecLayout { size_t S; FfnOff P; MabOff M1, M2; FfnOff D; };
+
 struct ParamLayout {
   // offsets (in floats) of each tensor inside the flat parameter vector
   std::vector<size_t> W_u, W_e, W_m, a_s, a_d;
   size_t W_1 = 0, b_1 = 0, w_2 = 0, b_2 = 0, total = 0;
   std::vector<int> d_in, de_in;
+  bool dec = false;
+  DecLayout D{};
+  int head_in = 0;          // W_1 columns: d (mean readout) or k·d (decoder)
 };
 ParamLayout make_layout(const occu_config &c);
 
@@ -52,6 +61,8 @@ struct Workspace {
   DevBuf tcpart;           // tensor-core aggregation: boundary-segment partials
   DevBuf dpart;            // per-warp [da_s; da_d] partials
   DevBuf anf[2], aef[2], acsr[2];   // occu_predict_async: double-buffered input staging
+  DevBuf dT, dZ;           // decoder readout: per-node FFN hidden / output rows [N][d]
+  DevBuf dprep;            // decoder readout: folded key map M [d][16] and offsets c [16]
   void release_all();
 };
 
@@ -213,6 +224,14 @@ int launch_permute_rows(const occu_ctx *ctx, const float *src, const int32_t *id
 // gather_segsum_kernel (row min(u1 - 1, 8c + 7) holds graph b's sum over chunk c).
 int launch_readout_head(const occu_ctx *ctx, const DevCsr &csr, const float *h, bool chunked,
                         const float *params, float *r, float *c, float *yhat, cudaStream_t st);
+// NEXT-2 readout (kernels_decoder.cu): Z = FFN(h_L) on tensor cores (T = ReLU(h W1ᵀ + b1),
+// Z = T W2ᵀ + b2), then per graph the k-seed attention pool over Z, the MAB / SAB / FFN tail
+// and the head; r receives the flattened decoder output [B][k·d].
+int launch_set_decoder(const occu_ctx *ctx, const DevCsr &csr, const float *hL, float *T, float *Z,
+                       float *r, float *c, float *yhat, cudaStream_t st);
+// Row-GEMM out = act(A Wᵀ + bias) over R rows on tensor cores with a prebuilt image (kernels_tc.cu).
+int launch_bias_tc(const occu_ctx *ctx, const float *A, int K, int R, int wkind, int layer,
+                   const float *bias, bool relu, float *out, const char *name, cudaStream_t st);
 
 struct BwdLayerArgs {
   int layer;

@@ -47,7 +47,7 @@ void Workspace::release_all() {
   DevBuf *bufs[] = {&node_feat, &edge_feat, &targets, &out_occ, &csr, &e0, &g, &r, &c, &yhat,
                     &dy, &dc, &dr, &dh, &dhprev, &dP, &MG, &DV, &DZ, &deA, &deB, &dalpha,
                     &dpq, &partial, &loss, &tcpart, &dpart, &rpart, &anf[0], &anf[1],
-                    &aef[0], &aef[1], &acsr[0], &acsr[1]};
+                    &aef[0], &aef[1], &acsr[0], &acsr[1], &dT, &dZ, &dprep};
   for (DevBuf *b : bufs) b->release();
   for (auto *v : {&hbar, &p, &q, &e, &h, &gs})
     for (DevBuf &b : *v) b.release();
@@ -163,6 +163,15 @@ occu_status validate_cfg(const occu_config *c) {
   if (c->prec == OCCU_BF16 && !(c->F_n <= 128 && (c->F_e <= 16 || c->F_e % 64 == 0)))
     return fail(nullptr, OCCU_EINVAL, "OCCU_BF16 needs F_n <= 128 and F_e <= 16 or a multiple of 64");
   if (!(c->slope > 0.f && c->slope < 1.f)) return fail(nullptr, OCCU_EINVAL, "slope must be in (0,1)");
+  if (c->readout != OCCU_READOUT_MEAN && c->readout != OCCU_READOUT_SET_DECODER)
+    return fail(nullptr, OCCU_EINVAL, "readout must be MEAN or SET_DECODER");
+  if (c->readout == OCCU_READOUT_SET_DECODER) {
+    if (c->prec != OCCU_FP32 || c->F_n > 128)
+      return fail(nullptr, OCCU_EINVAL, "the Set-Transformer decoder readout runs in OCCU_FP32 on the tensor-core path");
+    if (c->k < 1 || c->k > 8 || !(c->heads == 1 || c->heads == 2 || c->heads == 4 || c->heads == 8) ||
+        c->k * c->heads > 16 || c->d % c->heads)
+      return fail(nullptr, OCCU_EINVAL, "decoder: k in [1,8], heads in {1,2,4,8}, k*heads <= 16");
+  }
   return OCCU_OK;
 }
 
@@ -241,7 +250,8 @@ occu_status forward(occu_ctx *ctx, const DevCsr &csr, const float *nf, const flo
   // Tensor-core path fusions: a1's edge permutation folded into the layer-1 edge kernel,
   // and the readout's node sums folded into the last aggregation (chunk partials).
   const bool fuse_e0 = tc && c.F_e <= 16;
-  const bool fuse_ro = tc && (bf || ctx->path == 0);
+  const bool dec = c.readout == OCCU_READOUT_SET_DECODER;
+  const bool fuse_ro = tc && (bf || ctx->path == 0) && !dec;
   if (!fuse_e0) LK(launch_permute_rows(ctx, ef, csr.in_eid, csr.E, c.F_e, w.e0.as<float>(), s), "permute e0");
   if (tc) LK(tc_prepare_weights(ctx, s), "weight images");
   float *rpart = nullptr;
@@ -290,9 +300,19 @@ occu_status forward(occu_ctx *ctx, const DevCsr &csr, const float *nf, const flo
       LK(launch_forward_layer(ctx, csr, a, s), "forward layer");
     }
   }
-  LK(launch_readout_head(ctx, csr, fuse_ro ? rpart : w.h[c.L - 1].as<float>(), fuse_ro, P,
-                         w.r.as<float>(), w.c.as<float>(), w.yhat.as<float>(), s),
-     "readout/head");
+  if (dec) {
+    // NEXT-2: Set-Transformer decoder per graph, head on the flattened k·d output
+    CK(w.dT.ensure(size_t(csr.N) * c.d * 4), "alloc decoder scratch");
+    CK(w.dZ.ensure(size_t(csr.N) * c.d * 4), "alloc decoder scratch");
+    CK(w.r.ensure(size_t(csr.B) * c.k * c.d * 4), "alloc r");
+    LK(launch_set_decoder(ctx, csr, w.h[c.L - 1].as<float>(), w.dT.as<float>(), w.dZ.as<float>(),
+                          w.r.as<float>(), w.c.as<float>(), w.yhat.as<float>(), s),
+       "set decoder");
+  } else {
+    LK(launch_readout_head(ctx, csr, fuse_ro ? rpart : w.h[c.L - 1].as<float>(), fuse_ro, P,
+                           w.r.as<float>(), w.c.as<float>(), w.yhat.as<float>(), s),
+       "readout/head");
+  }
   ctx->h_last_stored = !fuse_ro || save_all;
   ctx->last_csr = csr;
   ctx->have_forward = true;
@@ -346,6 +366,8 @@ occu_status grads_impl(occu_ctx *ctx, const occu_batch *batch, const float *targ
   if (!batch || !batch->csr || !targets) return fail(ctx, OCCU_EINVAL, "batch/targets NULL");
   if (batch->global_num_graphs < batch->csr->num_graphs)
     return fail(ctx, OCCU_EINVAL, "global_num_graphs < local num_graphs");
+  if (ctx->cfg.readout == OCCU_READOUT_SET_DECODER)
+    return fail(ctx, OCCU_EINVAL, "the Set-Transformer decoder readout is inference-only in this build");
   ctx->launches = 0;
   if ((st = resolve_csr(ctx, batch->csr, csr)) != OCCU_OK) return st;
   if ((st = stage_inputs(ctx, csr, batch->node_feat, batch->edge_feat, targets, stg)) != OCCU_OK)
@@ -775,6 +797,8 @@ occu_status occu_set_kernel_path(occu_ctx *ctx, int path) {
     return fail(ctx, OCCU_EINVAL, "OCCU_BF16 runs on kernel path 0 only");
   if (ctx->cfg.msg == OCCU_MSG_NEIGHBOR_SOFTMAX && path != 0)
     return fail(ctx, OCCU_EINVAL, "reading B (NEIGHBOR_SOFTMAX) runs on kernel path 0 only");
+  if (ctx->cfg.readout == OCCU_READOUT_SET_DECODER && path != 0)
+    return fail(ctx, OCCU_EINVAL, "the decoder readout runs on kernel path 0 only");
   ctx->path = path;
   return OCCU_OK;
 }
@@ -807,7 +831,7 @@ occu_status occu_get_tensor(occu_ctx *ctx, int32_t which, int32_t layer, void *h
       if (layer == ctx->cfg.L - 1 && !ctx->h_last_stored)
         return fail(ctx, OCCU_ENOTREADY, "last-layer h not stored (set keep_intermediates)");
       src = w.h[layer].ptr; need = size_t(c.N) * d * 4; break;
-    case OCCU_T_R: src = w.r.ptr; need = size_t(c.B) * d * 4; break;
+    case OCCU_T_R: src = w.r.ptr; need = size_t(c.B) * ctx->layout.head_in * 4; break;   // [B][d] or [B][k·d]
     case OCCU_T_YHAT: src = w.yhat.ptr; need = size_t(c.B) * 4; break;
     default: return fail(ctx, OCCU_EINVAL, "unknown tensor");
   }

@@ -28,7 +28,28 @@ ParamLayout make_layout(const occu_config &c) {
     L.a_s.push_back(off); off += c.d;
     L.a_d.push_back(off); off += c.d;
   }
-  L.W_1 = off; off += size_t(c.d_h) * c.d;
+  L.head_in = c.d;
+  if (c.readout == OCCU_READOUT_SET_DECODER) {
+    const size_t d = size_t(c.d), dd = d * d;
+    L.dec = true;
+    auto ffn = [&](FfnOff &f) {
+      f.W1 = off; off += dd; f.b1 = off; off += d; f.W2 = off; off += dd; f.b2 = off; off += d;
+    };
+    L.D.S = off; off += size_t(c.k) * d;
+    ffn(L.D.P);
+    for (MabOff *m : {&L.D.M1, &L.D.M2}) {
+      m->Wq = off; off += dd; m->bq = off; off += d;
+      m->Wk = off; off += dd; m->bk = off; off += d;
+      m->Wv = off; off += dd; m->bv = off; off += d;
+      m->Wo = off; off += dd; m->bo = off; off += d;
+      m->ln1_g = off; off += d; m->ln1_b = off; off += d;
+      ffn(m->F);
+      m->ln2_g = off; off += d; m->ln2_b = off; off += d;
+    }
+    ffn(L.D.D);
+    L.head_in = c.k * c.d;
+  }
+  L.W_1 = off; off += size_t(c.d_h) * L.head_in;
   L.b_1 = off; off += c.d_h;
   L.w_2 = off; off += c.d_h;
   L.b_2 = off; off += 1;
@@ -56,11 +77,35 @@ void init_flat(const occu_config &c, uint64_t seed, std::vector<float> &out) {
     ts.push_back({L.a_s[i], size_t(c.d), 2 * c.d});
     ts.push_back({L.a_d[i], size_t(c.d), 2 * c.d});
   }
-  ts.push_back({L.W_1, size_t(c.d_h) * c.d, c.d});
-  ts.push_back({L.b_1, size_t(c.d_h), c.d});
+  if (L.dec) {
+    // fan_in -1: constant 1 (LayerNorm gain), 0: constant 0 (LayerNorm bias)
+    const size_t d = size_t(c.d), dd = d * d;
+    auto ffn = [&](const FfnOff &f) {
+      ts.push_back({f.W1, dd, c.d}); ts.push_back({f.b1, d, c.d});
+      ts.push_back({f.W2, dd, c.d}); ts.push_back({f.b2, d, c.d});
+    };
+    ts.push_back({L.D.S, size_t(c.k) * d, c.d});
+    ffn(L.D.P);
+    for (const MabOff *m : {&L.D.M1, &L.D.M2}) {
+      for (size_t w : {m->Wq, m->Wk, m->Wv, m->Wo}) {
+        ts.push_back({w, dd, c.d});
+        ts.push_back({w + dd, d, c.d});          // its bias follows it
+      }
+      ts.push_back({m->ln1_g, d, -1}); ts.push_back({m->ln1_b, d, 0});
+      ffn(m->F);
+      ts.push_back({m->ln2_g, d, -1}); ts.push_back({m->ln2_b, d, 0});
+    }
+    ffn(L.D.D);
+  }
+  ts.push_back({L.W_1, size_t(c.d_h) * L.head_in, L.head_in});
+  ts.push_back({L.b_1, size_t(c.d_h), L.head_in});
   ts.push_back({L.w_2, size_t(c.d_h), c.d_h});
   ts.push_back({L.b_2, 1, c.d_h});
   for (const T &t : ts) {
+    if (t.fan_in <= 0) {
+      for (size_t j = 0; j < t.n; ++j) out[t.off + j] = t.fan_in < 0 ? 1.f : 0.f;
+      continue;
+    }
     const double bound = 1.0 / sqrt(double(t.fan_in));
     for (size_t j = 0; j < t.n; ++j) {
       const uint64_t z = splitmix64_at(seed, t.off + j);
@@ -88,10 +133,12 @@ bool write_file(const char *path, const char magic[8], const occu_config &c,
     err = std::string("cannot open ") + path + " for writing";
     return false;
   }
-  uint32_t hdr[8] = {1u, uint32_t(c.L), uint32_t(c.F_n), uint32_t(c.F_e), uint32_t(c.d),
+  const bool v2 = c.readout == OCCU_READOUT_SET_DECODER;
+  uint32_t hdr[8] = {v2 ? 2u : 1u, uint32_t(c.L), uint32_t(c.F_n), uint32_t(c.F_e), uint32_t(c.d),
                      uint32_t(c.d_h), uint32_t(c.aggr), uint32_t(c.msg)};
+  const uint32_t ext[3] = {uint32_t(c.readout), uint32_t(c.k), uint32_t(c.heads)};
   bool ok = fwrite(magic, 1, 8, f) == 8 && fwrite(hdr, 4, 8, f) == 8 &&
-            fwrite(&c.slope, 4, 1, f) == 1;
+            fwrite(&c.slope, 4, 1, f) == 1 && (!v2 || fwrite(ext, 4, 3, f) == 3);
   uint64_t h = 0xCBF29CE484222325ull;
   for (auto &ch : chunks) {
     ok = ok && fwrite(ch.first, 1, ch.second, f) == ch.second;
@@ -120,18 +167,21 @@ occu_status read_file(const char *path, const char magic[8], const occu_config &
   size_t n;
   while ((n = fread(buf, 1, sizeof buf, f)) > 0) raw.insert(raw.end(), buf, buf + n);
   fclose(f);
-  const size_t hdr = 8 + 32 + 4;
+  const bool v2 = c.readout == OCCU_READOUT_SET_DECODER;
+  const size_t hdr = 8 + 32 + 4 + (v2 ? 12 : 0);
   if (raw.size() < hdr + 8 || memcmp(raw.data(), magic, 8) != 0) {
     err = "bad magic or truncated file";
     return OCCU_EFORMAT;
   }
-  uint32_t h[8];
+  uint32_t h[8], ext[3] = {0, 0, 0};
   memcpy(h, raw.data() + 8, 32);
   float slope;
   memcpy(&slope, raw.data() + 40, 4);
-  if (h[0] != 1u || int(h[1]) != c.L || int(h[2]) != c.F_n || int(h[3]) != c.F_e ||
+  if (v2) memcpy(ext, raw.data() + 44, 12);
+  if (h[0] != (v2 ? 2u : 1u) || int(h[1]) != c.L || int(h[2]) != c.F_n || int(h[3]) != c.F_e ||
       int(h[4]) != c.d || int(h[5]) != c.d_h || int(h[6]) != c.aggr || int(h[7]) != c.msg ||
-      slope != c.slope) {
+      slope != c.slope ||
+      (v2 && (int(ext[0]) != c.readout || int(ext[1]) != c.k || int(ext[2]) != c.heads))) {
     err = "file config does not match the context config";
     return OCCU_EINVAL;
   }

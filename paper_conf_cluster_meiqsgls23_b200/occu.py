@@ -44,7 +44,8 @@ class OccuError(RuntimeError):
 class Config(C.Structure):
     _fields_ = [("L", C.c_int32), ("F_n", C.c_int32), ("F_e", C.c_int32), ("d", C.c_int32),
                 ("d_h", C.c_int32), ("aggr", C.c_int32), ("msg", C.c_int32), ("prec", C.c_int32),
-                ("slope", C.c_float)]
+                ("slope", C.c_float), ("readout", C.c_int32), ("k", C.c_int32),
+                ("heads", C.c_int32)]
 
 
 class GraphView(C.Structure):
@@ -139,9 +140,13 @@ def _ptr(x):
     return x.data_ptr(), bool(x.is_cuda), x
 
 
+READOUT_MEAN, READOUT_SET_DECODER = 0, 1
+
+
 def config(L=3, F_n=80, F_e=4, d=128, d_h=None, aggr=AGGR_SUM, msg=MSG_CHANNEL_SOFTMAX,
-           prec=FP32, slope=0.01):
-    return Config(L, F_n, F_e, d, d if d_h is None else d_h, aggr, msg, prec, slope)
+           prec=FP32, slope=0.01, readout=READOUT_MEAN, k=4, heads=4):
+    return Config(L, F_n, F_e, d, d if d_h is None else d_h, aggr, msg, prec, slope, readout,
+                  k if readout else 0, heads if readout else 0)
 
 
 def num_params(cfg: Config) -> int:
