@@ -260,6 +260,8 @@ def main():
     ap.add_argument("--ref-graphs", type=int, default=32)
     ap.add_argument("--no-train", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--no-cfg3", action="store_true", help="skip the CFG3 training line")
+    ap.add_argument("--cfg3-graphs", type=int, default=512, help="CFG3 graphs per rank")
     ap.add_argument("--no-flush", action="store_true")
     ap.add_argument("--no-bf16", action="store_true", help="skip the OCCU_BF16 inference line")
     ap.add_argument("--path", type=int, default=0, help="0: tcgen05 3xTF32 (default), 1: SIMT FP32")
@@ -548,7 +550,8 @@ def main():
         talg = train_algorithmic_bytes(N, E, B, d, rrows=rrows)
         tk, troof = kernel_table(tprof, talg, load_traffic())
         tot_alg = sum(v for k, v in talg.items() if k in tprof)
-        train = {"value": gB / (tms * 1e-3), "unit": "graphs/s", "ms_per_step": tms,
+        train = {"workload": "CFG2 graphs (256 ResNet-50 training graphs per rank), one training step",
+                 "value": gB / (tms * 1e-3), "unit": "graphs/s", "ms_per_step": tms,
                  "global_batch": gB, "gpu_launches": tl, "loss_after": loss,
                  "roofline": troof,
                  "step_algorithmic_bytes": tot_alg,
@@ -585,6 +588,59 @@ def main():
                              "kernel_ms_per_step": {k: v[0] / args.steps for k, v in bprof.items()}}
             del mb
 
+    # ---- CFG3 (BASELINE.json configs[2]): 512 BERT-base / GPT-2 training graphs per rank,
+    # one full training step (forward with saves, MSE, backward, [allreduce,] Adam), FP32 and BF16
+    train_cfg3 = None
+    if not args.no_train and not args.no_cfg3 and args.path == 0:
+        b3 = configs.cfg3(args.cfg3_graphs)
+        B3, N3, E3 = b3.num_graphs, b3.num_nodes, b3.num_edges
+        csr3 = model.to_device(occu.pack(b3.graphs))
+        nf3 = torch.from_numpy(b3.node_feat).to(dev)
+        ef3 = torch.from_numpy(b3.edge_feat).to(dev)
+        yt3 = torch.from_numpy(b3.targets).to(dev)
+        rr3 = readout_rows(b3.graphs)
+        gB3 = B3 * world
+        train_cfg3 = {"workload": "CFG3 (BASELINE.json configs[2]): %d transformer training graphs "
+                                  "per rank (half BERT-base, half GPT-2)" % B3,
+                      "graphs_per_rank": B3, "nodes_per_rank": N3, "edges_per_rank": E3,
+                      "global_batch": gB3}
+        for prec, sa, key in ((occu.FP32, 4, "f32"), (occu.BF16, 2, "bf16")):
+            if prec == occu.BF16 and args.no_bf16:
+                continue
+            m3 = occu.Model(occu.config(L=3, F_n=80, F_e=4, d=128, prec=prec), device=local,
+                            stream=stream.cuda_stream)
+            m3.init_weights(42)
+            if pg and world > 1:
+                uid = [occu.Model.nccl_unique_id() if rank == 0 else None]
+                pg.broadcast_object_list(uid, src=0)
+                m3.dist_init(rank, world, uid[0])
+            st3 = lambda: m3.train_step(csr3, nf3, ef3, yt3, 1e-4, global_num_graphs=gB3,
+                                        want_loss=False)
+            loss0 = m3.train_step(csr3, nf3, ef3, yt3, 1e-4, global_num_graphs=gB3)
+            with ClockSampler(local) as clk3:
+                timed(st3, args.warmup, mdl=m3)
+                bar()
+                t3, l3 = timed(st3, args.steps, mdl=m3)
+                bar()
+                timed(st3, args.steps, profile=True, mdl=m3)
+                bar()
+            ms3 = max_over_ranks(float(np.sum(t3)) / args.steps)
+            a3 = train_algorithmic_bytes(N3, E3, B3, d, rrows=rr3, sa=sa)
+            p3 = m3.profile()
+            k3, r3 = kernel_table(p3, a3, load_traffic() if sa == 4 else {})
+            tot3 = sum(v for k, v in a3.items() if k in p3)
+            train_cfg3[key] = {
+                "value": gB3 / (ms3 * 1e-3), "unit": "graphs/s", "ms_per_step": ms3,
+                "dtype": key, "gpu_launches": l3, "roofline": r3,
+                "step_algorithmic_bytes": tot3,
+                "step_frac_of_hbm": tot3 / (ms3 * 1e-3) / 1e9 / peaks["hbm_gbs"],
+                "loss_first": loss0,
+                "loss_after": m3.train_step(csr3, nf3, ef3, yt3, 1e-4, global_num_graphs=gB3),
+                "clocks": clk3.summary(),
+                "kernel_ms_per_step": {k: v["ms_per_step"] for k, v in k3.items()}, "kernels": k3}
+            del m3
+        del nf3, ef3, yt3, csr3
+
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu:
         cpu = cpu_baseline_sample()
@@ -614,6 +670,7 @@ def main():
             "readingb": readingb,
             "decoder": decoder,
             "train": train,
+            "train_cfg3": train_cfg3,
             "cpu_baseline": cpu,
         }
         print(json.dumps(line), flush=True)
