@@ -3,7 +3,9 @@
 Layout (SURVEY §8(b) "Weights file"; shapes from P141-P149 read as in
 DESIGN.md R1-R6): for each ANEE layer i = 1..L
     W_u[d][d_in]  W_e[d][d_e_in]  W_m[d][d]  a_s[d]  a_d[d]
-with d_in = F_n, d_e_in = F_e for i = 1 and d otherwise; with the Set-Transformer
+with d_in = F_n, d_e_in = F_e for i = 1 and d otherwise; then per Graphormer layer j
+(graphormer > 0) G{j}_ ln1_g ln1_b Wq bq Wk bk Wv bv Wo bo ln2_g ln2_b
+F_W1 F_b1 F_W2 F_b2; with the Set-Transformer
 decoder readout (readout = 1, R30-R34) the decoder's
 parameters follow (seeds S[k][d]; the pre-pooling FFN P_*; the two MABs M1_*, M2_* each
 Wq bq Wk bk Wv bv Wo bo ln1_g ln1_b F_W1 F_b1 F_W2 F_b2 ln2_g ln2_b; the final FFN D_*);
@@ -16,8 +18,9 @@ biases 0 (PyTorch's LayerNorm init).  The C library's ``occu_init_weights`` impl
 same rule independently.
 
 File: b"OCCUW001", u32[8] = (version, L, F_n, F_e, d, d_h, aggr, msg), f32 slope,
-[version 2 only: u32[3] = (readout, k, heads)], f32 payload (flat, file order), u64
-FNV-1a of the payload bytes.  Version 1 = mean readout, version 2 = decoder readout.
+[version 2: u32[3] = (readout, k, heads); version 3: u32[4] = (readout, k, heads,
+graphormer)], f32 payload (flat, file order), u64 FNV-1a of the payload bytes.  Version 1 =
+mean readout, version 2 = decoder readout, version 3 = Graphormer layers (any readout).
 No method arithmetic lives here.
 """
 from __future__ import annotations
@@ -48,7 +51,8 @@ class ModelConfig:
     slope: float = 0.01
     readout: int = 0        # 0: segmented mean (a7), 1: Set-Transformer decoder (NEXT-2)
     k: int = 4              # decoder seeds
-    heads: int = 4          # decoder attention heads
+    heads: int = 4          # decoder / Graphormer attention heads
+    graphormer: int = 0     # Graphormer layers after the ANEE rounds (NEXT-3)
 
 
 def param_specs(cfg: ModelConfig):
@@ -66,9 +70,15 @@ def param_specs(cfg: ModelConfig):
         ]
     d = cfg.d
     hin = d
+    # fan_in -1: constant 1 (LayerNorm gain), 0: constant 0 (LayerNorm bias)
+    lin = lambda p: [(f"{p}W1", (d, d), d), (f"{p}b1", (d,), d), (f"{p}W2", (d, d), d), (f"{p}b2", (d,), d)]
+    for j in range(cfg.graphormer):          # Graphormer layers (NEXT-3)
+        g = f"G{j}_"
+        specs += [(f"{g}ln1_g", (d,), -1), (f"{g}ln1_b", (d,), 0)]
+        for w in ("q", "k", "v", "o"):
+            specs += [(f"{g}W{w}", (d, d), d), (f"{g}b{w}", (d,), d)]
+        specs += [(f"{g}ln2_g", (d,), -1), (f"{g}ln2_b", (d,), 0)] + lin(f"{g}F_")
     if cfg.readout == 1:
-        # fan_in -1: constant 1 (LayerNorm gain), 0: constant 0 (LayerNorm bias)
-        lin = lambda p: [(f"{p}W1", (d, d), d), (f"{p}b1", (d,), d), (f"{p}W2", (d, d), d), (f"{p}b2", (d,), d)]
         specs += [("S", (cfg.k, d), d)] + lin("P_")
         for m in ("M1_", "M2_"):
             for w in ("q", "k", "v", "o"):
@@ -138,11 +148,14 @@ def write_weights(path: str, cfg: ModelConfig, flat: np.ndarray) -> None:
     payload = flat.tobytes()
     with open(path, "wb") as f:
         f.write(MAGIC)
-        f.write(struct.pack("<8I", 2 if cfg.readout else VERSION, cfg.L, cfg.F_n, cfg.F_e, cfg.d,
+        version = 3 if cfg.graphormer else (2 if cfg.readout else VERSION)
+        f.write(struct.pack("<8I", version, cfg.L, cfg.F_n, cfg.F_e, cfg.d,
                             cfg.d_h, cfg.aggr, cfg.msg))
         f.write(struct.pack("<f", cfg.slope))
-        if cfg.readout:
+        if version == 2:
             f.write(struct.pack("<3I", cfg.readout, cfg.k, cfg.heads))
+        elif version == 3:
+            f.write(struct.pack("<4I", cfg.readout, cfg.k, cfg.heads, cfg.graphormer))
         f.write(payload)
         f.write(struct.pack("<Q", fnv1a64(payload)))
 

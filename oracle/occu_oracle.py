@@ -15,7 +15,9 @@ Computation (per ANEE layer i, P139-P151; R1-R9):
     e^i_l = σ(α_l · (W_e e^{i-1}_l))                                P145 (R2, R3)
     f(u',l') = Softmax_channels(W_m e^i_l') ⊙ h̄_u'                  P149 (R4, reading A)
     h^i_u = LeakyReLU(Σ_{l'=(u',u)} f(u',l'))                       P149 (R8, R9)
-then per-graph mean readout (north_star; R11) and the MLP head (P125; R12),
+optionally Graphormer layers per graph (P153-P157, NEXT-3; R35-R37), then the per-graph
+mean readout (north_star; R11) or the Set-Transformer decoder (P159-P205, NEXT-2; R30-R34)
+and the MLP head (P125; R12),
 MSE loss (P209-P213), Adam (P273; R16).
 
 Parity status: every function here is pinned by tests in tests/test_oracle.py
@@ -89,6 +91,9 @@ def read_weights(path):
     if version == 2:                      # Set-Transformer decoder readout (NEXT-2)
         cfg["readout"], cfg["k"], cfg["heads"] = struct.unpack_from("<3I", raw, 44)
         hdr = 56
+    elif version == 3:                    # + Graphormer layers (NEXT-3)
+        cfg["readout"], cfg["k"], cfg["heads"], cfg["graphormer"] = struct.unpack_from("<4I", raw, 44)
+        hdr = 60
     flat = np.frombuffer(raw, dtype="<f4", offset=hdr, count=(len(raw) - hdr - 8) // 4)
     return cfg, unflatten(cfg, flat.astype(np.float64))
 
@@ -103,10 +108,17 @@ def param_shapes(cfg):
                 (f"W_m{i}", (cfg["d"], cfg["d"])), (f"a_s{i}", (cfg["d"],)),
                 (f"a_d{i}", (cfg["d"],))]
     d, hin = cfg["d"], cfg["d"]
+    ffn = lambda p: [(p + "W1", (d, d)), (p + "b1", (d,)), (p + "W2", (d, d)), (p + "b2", (d,))]
+    for j in range(cfg.get("graphormer", 0)):
+        # Graphormer layer j (P153-P157; R35-R37): LN1, MHA, LN2, FFN
+        g = f"G{j}_"
+        out += [(g + "ln1_g", (d,)), (g + "ln1_b", (d,))]
+        for w in "qkvo":
+            out += [(g + "W" + w, (d, d)), (g + "b" + w, (d,))]
+        out += [(g + "ln2_g", (d,)), (g + "ln2_b", (d,))] + ffn(g + "F_")
     if cfg.get("readout", 0) == 1:
         # Set-Transformer decoder (P159-P205; R30-R34): seeds, pre-pooling FFN,
         # MAB1 (PMA), MAB2 (SAB), final FFN; the head then reads the flattened k x d output
-        ffn = lambda p: [(p + "W1", (d, d)), (p + "b1", (d,)), (p + "W2", (d, d)), (p + "b2", (d,))]
         out += [("S", (cfg["k"], d))] + ffn("P_")
         for m in ("M1_", "M2_"):
             for w in "qkvo":
@@ -226,8 +238,8 @@ def forward_anee(params, cfg, pk, node_feat, edge_feat):
         h, e = lay["h"], lay["e"]
     out = dict(layers=layers, e0=np.asarray(edge_feat, np.float64)[pk["in_eid"].astype(np.int64)],
                h0=np.asarray(node_feat, np.float64))
-    if cfg.get("readout", 0) == 1:         # the decoder readout follows in forward()
-        return out
+    if cfg.get("readout", 0) == 1 or cfg.get("graphormer", 0) > 0:
+        return out                        # Graphormer layers / the decoder follow in forward()
     n_b = np.diff(pk["node_off"].astype(np.int64))
     # north_star: segmented per-graph readout, mean over nodes (R11)
     r = segment_sum(h, pk["node_graph"].astype(np.int64), pk["num_graphs"]) / n_b[:, None]
@@ -345,20 +357,43 @@ def set_decoder(H, params, heads):
     return ffn(sab, params, "D_")
 
 
+def graphormer_layer(H, params, j, heads):
+    """Graphormer layer j over one graph's node states H [n, d] (P153-P157; R35-R37):
+        h̄ = MHA(LN(h)) + h,    h' = FFN(LN(h̄)) + h̄
+    with self-attention over all n nodes of the graph (MHA(X, X, X), R32 heads)."""
+    g = f"G{j}_"
+    X = layer_norm(H, params[g + "ln1_g"], params[g + "ln1_b"])
+    Hb = mha(X, X, params, g, heads) + H
+    Y = layer_norm(Hb, params[g + "ln2_g"], params[g + "ln2_b"])
+    return ffn(Y, params, g + "F_") + Hb
+
+
 def forward(params, cfg, pk, node_feat, edge_feat):
-    """forward_anee + readout: the segmented mean (a7) or, with cfg["readout"] == 1, the
-    Set-Transformer decoder per graph (NEXT-2), then the MLP head on its flattened output."""
+    """forward_anee, then cfg["graphormer"] Graphormer layers per graph (NEXT-3), then the
+    readout: the segmented mean (a7) or, with cfg["readout"] == 1, the Set-Transformer decoder
+    per graph (NEXT-2); then the MLP head on the (flattened) readout."""
     f = forward_anee(params, cfg, pk, node_feat, edge_feat)
-    if cfg.get("readout", 0) != 1:
+    G = cfg.get("graphormer", 0)
+    if cfg.get("readout", 0) != 1 and G == 0:
         return f
     hL = f["layers"][-1]["h"]
     off = pk["node_off"].astype(np.int64)
-    D = np.stack([set_decoder(hL[off[b]:off[b + 1]], params, cfg["heads"])
-                  for b in range(pk["num_graphs"])])
-    r = D.reshape(pk["num_graphs"], -1)
+    B = pk["num_graphs"]
+    gph = []
+    for j in range(G):
+        hL = np.concatenate([graphormer_layer(hL[off[b]:off[b + 1]], params, j, cfg["heads"])
+                             for b in range(B)])
+        gph.append(hL)
+    f["gph"] = gph
+    if cfg.get("readout", 0) == 1:
+        D = np.stack([set_decoder(hL[off[b]:off[b + 1]], params, cfg["heads"]) for b in range(B)])
+        f["dec"] = D
+        r = D.reshape(B, -1)
+    else:                                 # segmented mean readout (R11)
+        r = segment_sum(hL, pk["node_graph"].astype(np.int64), B) / np.diff(off)[:, None]
     c = r @ params["W_1"].T + params["b_1"]
     o = leaky_relu(c, cfg["slope"])
-    f.update(dec=D, r=r, c=c, o=o, yhat=o @ params["w_2"] + params["b_2"][0])
+    f.update(r=r, c=c, o=o, yhat=o @ params["w_2"] + params["b_2"][0])
     return f
 
 
@@ -380,8 +415,8 @@ def mse_loss(yhat, y, global_batch=None):
 def backward(params, cfg, pk, fwd, y, global_batch=None, dsig=None):
     """dsig(layer dict) -> σ'(y) per edge and channel; default e'(1 - e') (exact
     derivative of σ at y = α z).  backward_bf16 passes e'·σ(-α z) (R28)."""
-    if cfg.get("readout", 0) == 1:
-        raise NotImplementedError("training with the decoder readout (NEXT-2) is inference-only here")
+    if cfg.get("readout", 0) == 1 or cfg.get("graphormer", 0) > 0:
+        raise NotImplementedError("training through the decoder / Graphormer layers is not built (NEXT-2/3 are inference-only)")
     slope = cfg["slope"]
     B = pk["num_graphs"]
     nb = B if global_batch is None else global_batch

@@ -645,3 +645,152 @@ def test_decoder_readout_node_permutation_and_batching_invariance():
         efs.append(b.edge_feat[eoff[g]:eoff[g + 1]])
     y2 = oracle.predict(p, c, graphs, np.concatenate(nfs), np.concatenate(efs))
     assert np.allclose(y2, y, rtol=1e-12, atol=1e-14)
+
+
+# ------------------------------------------ NEXT-3: Graphormer layers (P153-P157)
+def gph_cfg(G=2, heads=4, d=16, L=2, readout=0, k=2):
+    c = cfg_dict(L=L, F_n=80, F_e=4, d=d, d_h=8)
+    c.update(readout=readout, k=k, heads=heads, graphormer=G)
+    return c
+
+
+def gph_params(c, seed):
+    wc = weights.ModelConfig(L=c["L"], F_n=c["F_n"], F_e=c["F_e"], d=c["d"], d_h=c["d_h"],
+                             readout=c["readout"], k=c["k"], heads=c["heads"],
+                             graphormer=c["graphormer"])
+    p = oracle.unflatten(c, weights.init_flat(wc, seed).astype(np.float64))
+    for i in range(c["L"]):
+        p[f"W_u{i}"] *= 4.0
+    rng = np.random.default_rng(seed)
+    for j in range(c["graphormer"]):              # non-trivial LayerNorm affine parameters
+        for ln in ("ln1", "ln2"):
+            p[f"G{j}_{ln}_g"] = 1.0 + 0.3 * rng.standard_normal(c["d"])
+            p[f"G{j}_{ln}_b"] = 0.2 * rng.standard_normal(c["d"])
+    return p
+
+
+def torch_graphormer(H, p, c, j):
+    """Independent Graphormer layer (P155, P157): pre-LN self-attention and FFN blocks with
+    residuals, built from torch's nn.LayerNorm and nn.MultiheadAttention (float64)."""
+    torch = pytest.importorskip("torch")
+    d, heads = c["d"], c["heads"]
+    T = lambda a: torch.tensor(a, dtype=torch.float64)
+    F = torch.nn.functional
+    g = f"G{j}_"
+    att = torch.nn.MultiheadAttention(d, heads, bias=True, batch_first=True, dtype=torch.float64)
+    ln1 = torch.nn.LayerNorm(d, eps=1e-5, dtype=torch.float64)
+    ln2 = torch.nn.LayerNorm(d, eps=1e-5, dtype=torch.float64)
+    with torch.no_grad():
+        att.in_proj_weight.copy_(torch.cat([T(p[g + "Wq"]), T(p[g + "Wk"]), T(p[g + "Wv"])]))
+        att.in_proj_bias.copy_(torch.cat([T(p[g + "bq"]), T(p[g + "bk"]), T(p[g + "bv"])]))
+        att.out_proj.weight.copy_(T(p[g + "Wo"]))
+        att.out_proj.bias.copy_(T(p[g + "bo"]))
+        ln1.weight.copy_(T(p[g + "ln1_g"])); ln1.bias.copy_(T(p[g + "ln1_b"]))
+        ln2.weight.copy_(T(p[g + "ln2_g"])); ln2.bias.copy_(T(p[g + "ln2_b"]))
+        h = T(H)
+        x = ln1(h)
+        a, _ = att(x[None], x[None], x[None], need_weights=False)
+        hb = a[0] + h
+        y = ln2(hb)
+        f = F.linear(F.relu(F.linear(y, T(p[g + "F_W1"]), T(p[g + "F_b1"]))), T(p[g + "F_W2"]), T(p[g + "F_b2"]))
+        return (f + hb).numpy()
+
+
+@pytest.mark.parametrize("G,heads,readout", [(2, 4, 0), (1, 2, 0), (2, 4, 1)])
+def test_graphormer_matches_torch_modules(G, heads, readout):
+    c = gph_cfg(G=G, heads=heads, readout=readout)
+    b = configs.random_dag_batch(4, 300 + G + heads, max_nodes=20, hub=True)
+    p = gph_params(c, 11 + G)
+    pk = oracle.pack(b.graphs)
+    f = oracle.forward(p, c, pk, b.node_feat, b.edge_feat)
+    off = pk["node_off"]
+    h = f["layers"][-1]["h"]
+    for j in range(G):
+        ref = np.concatenate([torch_graphormer(h[off[g]:off[g + 1]], p, c, j)
+                              for g in range(pk["num_graphs"])])
+        assert np.allclose(f["gph"][j], ref, rtol=1e-10, atol=1e-12), j
+        h = ref
+    if readout == 0:          # mean readout of the last Graphormer output, then the head
+        r = np.stack([h[off[g]:off[g + 1]].mean(axis=0) for g in range(pk["num_graphs"])])
+        y = oracle.leaky_relu(r @ p["W_1"].T + p["b_1"], c["slope"]) @ p["w_2"] + p["b_2"][0]
+        assert np.allclose(f["yhat"], y, rtol=1e-12, atol=1e-14)
+    else:                     # the decoder reads the Graphormer output
+        for g in range(pk["num_graphs"]):
+            assert np.allclose(f["dec"][g], torch_decoder(h[off[g]:off[g + 1]], p, c),
+                               rtol=1e-10, atol=1e-12)
+
+
+def test_graphormer_zero_output_maps_is_identity():
+    """With W_o = b_o = 0 and the FFN's W2 = b2 = 0 both residual branches vanish: the layer
+    is the identity, bitwise (P155, P157 residual form)."""
+    c = gph_cfg(G=2)
+    b = configs.random_dag_batch(3, 61, max_nodes=15)
+    p = gph_params(c, 4)
+    for j in range(2):
+        for n in ("Wo", "bo", "F_W2", "F_b2"):
+            p[f"G{j}_{n}"] = np.zeros_like(p[f"G{j}_{n}"])
+    pk = oracle.pack(b.graphs)
+    f = oracle.forward(p, c, pk, b.node_feat, b.edge_feat)
+    assert np.array_equal(f["gph"][1], f["layers"][-1]["h"])
+
+
+def test_graphormer_single_node_graph_closed_form():
+    """One node: attention over a single key is exactly 1, so MHA(x) = W_o (W_v x + b_v) + b_o
+    whatever W_q, W_k (bitwise invariance), and the layer has the closed form below."""
+    c = gph_cfg(G=1, heads=2)
+    p = gph_params(c, 8)
+    single = [(1, np.zeros(0, np.int32), np.zeros(0, np.int32))] * 3
+    nf = np.random.default_rng(5).normal(size=(3, 80))
+    ef = np.zeros((0, 4))
+    pk = oracle.pack(single)
+    f = oracle.forward(p, c, pk, nf, ef)
+    h = f["layers"][-1]["h"]
+    ln = lambda x, g, bb: (x - x.mean(-1, keepdims=True)) / np.sqrt(x.var(-1, keepdims=True) + 1e-5) * g + bb
+    x = ln(h, p["G0_ln1_g"], p["G0_ln1_b"])
+    hb = (x @ p["G0_Wv"].T + p["G0_bv"]) @ p["G0_Wo"].T + p["G0_bo"] + h
+    y = ln(hb, p["G0_ln2_g"], p["G0_ln2_b"])
+    ref = np.maximum(y @ p["G0_F_W1"].T + p["G0_F_b1"], 0) @ p["G0_F_W2"].T + p["G0_F_b2"] + hb
+    assert np.allclose(f["gph"][0], ref, rtol=1e-12, atol=1e-13)
+    q = dict(p)
+    q["G0_Wq"] = p["G0_Wq"] * 3.0 - 1.0
+    q["G0_Wk"] = -p["G0_Wk"]
+    q["G0_bk"] = p["G0_bk"] + 5.0
+    assert np.array_equal(oracle.forward(q, c, pk, nf, ef)["gph"][0], f["gph"][0])
+
+
+def test_graphormer_node_permutation_and_batching_invariance():
+    """Self-attention over a graph's node set is permutation-equivariant and never crosses
+    graphs: ŷ is invariant to relabelling nodes and equal batched vs one graph at a time."""
+    c = gph_cfg(G=2)
+    b = configs.random_dag_batch(5, 129, max_nodes=25, hub=True)
+    p = gph_params(c, 6)
+    y = oracle.predict(p, c, b.graphs, b.node_feat, b.edge_feat)
+    for g in range(b.num_graphs):
+        s = b.subset([g])
+        assert np.allclose(oracle.predict(p, c, s.graphs, s.node_feat, s.edge_feat), y[g:g + 1],
+                           rtol=1e-12, atol=1e-14)
+    rng = np.random.default_rng(18)
+    graphs, nfs, efs = [], [], []
+    noff = np.concatenate([[0], np.cumsum([g[0] for g in b.graphs])])
+    eoff = np.concatenate([[0], np.cumsum([len(g[1]) for g in b.graphs])])
+    for g, (n, s_, t_) in enumerate(b.graphs):
+        perm = rng.permutation(n)
+        inv = np.argsort(perm)
+        graphs.append((n, inv[s_].astype(np.int32), inv[t_].astype(np.int32)))
+        nfs.append(b.node_feat[noff[g]:noff[g + 1]][perm])
+        efs.append(b.edge_feat[eoff[g]:eoff[g + 1]])
+    y2 = oracle.predict(p, c, graphs, np.concatenate(nfs), np.concatenate(efs))
+    assert np.allclose(y2, y, rtol=1e-11, atol=1e-13)
+
+
+def test_graphormer_weights_file_v3_roundtrip(tmp_path):
+    c = gph_cfg(G=2, readout=1, k=3)
+    wc = weights.ModelConfig(L=c["L"], F_n=80, F_e=4, d=c["d"], d_h=c["d_h"], readout=1, k=3,
+                             heads=c["heads"], graphormer=2)
+    flat = weights.init_flat(wc, 42)
+    path = str(tmp_path / "w.bin")
+    weights.write_weights(path, wc, flat)
+    cf, p = oracle.read_weights(path)
+    assert cf["graphormer"] == 2 and cf["readout"] == 1 and cf["k"] == 3
+    assert np.array_equal(oracle.flatten(cf, p), flat.astype(np.float64))
+    assert np.all(p["G1_ln2_g"] == 1.0) and np.all(p["G0_ln1_b"] == 0.0)
