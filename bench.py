@@ -482,6 +482,54 @@ def main():
                            "head on the flattened 4 x 128 output (P159-P205)"}
         del md
 
+    # ---- NEXT-3: Graphormer layers (2 layers, 4 heads; P153-P157, P273) + mean readout, same batch
+    graphormer = None
+    if not args.no_bf16 and args.path == 0:
+        G_ = 2
+        mg = occu.Model(occu.config(L=3, F_n=80, F_e=4, d=128, heads=4, graphormer=G_),
+                        device=local, stream=stream.cuda_stream)
+        mg.init_weights(42)
+        outg = torch.empty_like(out)
+        inferg = lambda: mg.predict(csr, nf, ef, outg)
+        timed(inferg, args.warmup, mdl=mg)
+        bar()
+        tg_, lg_ = timed(inferg, args.steps, mdl=mg)
+        bar()
+        timed(inferg, args.steps, profile=True, mdl=mg)
+        bar()
+        msg_ = max_over_ranks(float(np.sum(tg_)) / args.steps)
+        algg = algorithmic_bytes(N, E, B, d)                  # h_L stored: unfused gather
+        Nd4 = 4 * N * d
+        algg["gph_ln"] = G_ * 2 * 2 * Nd4
+        algg["gph_qkv_tc"] = G_ * 3 * 2 * Nd4
+        algg["gph_out_tc"] = G_ * 3 * Nd4
+        algg["gph_ffn_tc"] = G_ * (2 * Nd4 + 3 * Nd4)
+        algg["gph_attn"] = G_ * 4 * Nd4                       # Q, K, V read once, O written
+        pg_ = mg.profile()
+        kg, roofg = kernel_table(pg_, algg, {})
+        nb = np.array([g_[0] for g_ in batch.graphs], np.float64)
+        attn_flops = G_ * float(np.sum(4.0 * nb * nb * d))    # QKᵀ + PV per layer: 4 n² d
+        attn_ms = pg_["gph_attn"][0] / args.steps if "gph_attn" in pg_ else None
+        tf32_peak = peaks["bf16_tflops"] * (1.1 / 2.25)         # guide's nominal tf32/bf16 ratio
+        attn_roof = None
+        if attn_ms:
+            ach = attn_flops / (attn_ms * 1e-3) / 1e12
+            attn_roof = {"kernel": "gph_attn", "bound": "tensor", "achieved": ach,
+                         "peak": tf32_peak, "unit": "TFLOP/s", "frac": ach / tf32_peak,
+                         "traffic": None, "algorithmic_flops_per_launch": attn_flops / G_,
+                         "avg_launch_ms": attn_ms / G_, "peak_kind": "measured bf16 x nominal tf32/bf16 (1.1/2.25)",
+                         "issued_mma_per_flop": 3,
+                         "note": "FP32 accuracy via the 3-product TF32 split: the tensor pipe issues 3x the "
+                                 "algorithmic flops (mma.sync m16n8k8)"}
+        graphormer = {"value": B * world / (msg_ * 1e-3), "unit": "graphs/s", "ms_per_step": msg_,
+                      "dtype": "f32", "gpu_launches": lg_, "roofline": roofg,
+                      "attention_roofline": attn_roof,
+                      "kernel_ms_per_step": {k_: v["ms_per_step"] for k_, v in kg.items()},
+                      "kernels": kg,
+                      "what": "ANEE x3 -> Graphormer x2 (pre-LN MHA over each graph's nodes, 4 heads, "
+                              "+ FFN) -> mean readout -> head (P153-P157)"}
+        del mg
+
     # ---- e2e through the public API with host buffers (pinned), pack included
     pin_nf = torch.from_numpy(batch.node_feat).pin_memory()
     pin_ef = torch.from_numpy(batch.edge_feat).pin_memory()
@@ -669,6 +717,7 @@ def main():
             "bf16": bf16,
             "readingb": readingb,
             "decoder": decoder,
+            "graphormer": graphormer,
             "train": train,
             "train_cfg3": train_cfg3,
             "cpu_baseline": cpu,

@@ -66,7 +66,12 @@ typedef enum { OCCU_READOUT_MEAN = 0, OCCU_READOUT_SET_DECODER = 1 } occu_readou
  * mean; default when the trailing fields are zero) or OCCU_READOUT_SET_DECODER (P159-P205,
  * NEXT-2: Decoder(H) = FFN(SAB(PMA_k(H))) per graph, k seeds, `heads` attention heads, the
  * head reading the flattened k·d output; OCCU_FP32, kernel path 0, inference only: training
- * returns OCCU_EINVAL); k in [1, 8], heads in {1, 2, 4, 8}, k·heads <= 16. */
+ * returns OCCU_EINVAL); k in [1, 8], heads in {1, 2, 4, 8}, k·heads <= 16.
+ * graphormer: number of Graphormer layers (P153-P157, NEXT-3; R35-R37) between the
+ * last ANEE round and the readout, h̄ = MHA(LN(h)) + h, h' = FFN(LN(h̄)) + h̄ with
+ * self-attention over each graph's own node set, `heads` heads (d / heads in {16, 32, 64});
+ * 0 = none (default).  OCCU_FP32, kernel path 0, inference only (training returns
+ * OCCU_EINVAL); graphormer in [0, 4]. */
 typedef struct {
   int32_t L, F_n, F_e, d, d_h;
   int32_t aggr;      /* occu_aggr */
@@ -74,7 +79,8 @@ typedef struct {
   int32_t prec;      /* occu_precision */
   float slope;
   int32_t readout;   /* occu_readout */
-  int32_t k, heads;  /* decoder seeds and heads (readout = OCCU_READOUT_SET_DECODER) */
+  int32_t k, heads;  /* decoder seeds; decoder / Graphormer attention heads */
+  int32_t graphormer; /* Graphormer layers (NEXT-3), 0 = none */
 } occu_config;
 
 /* One caller-owned input graph (host memory), local node ids. */
@@ -187,7 +193,8 @@ typedef enum {
   OCCU_T_E = 3,      /* [E][d]  layer l, in-CSR edge order */
   OCCU_T_H = 4,      /* [N][d]  layer l */
   OCCU_T_R = 5,      /* [B][d]  readout ([B][k·d] flattened decoder output with the decoder) */
-  OCCU_T_YHAT = 6    /* [B] */
+  OCCU_T_YHAT = 6,   /* [B] */
+  OCCU_T_GPH = 7     /* [N][d]  output of Graphormer layer l (NEXT-3) */
 } occu_tensor;
 /* Kernel path: 0 (default) = tcgen05 tensor cores (fp16x2-split GEMMs with
  * per-row power-of-two scaling, FP32 accumulation in TMEM) + CUDA-core

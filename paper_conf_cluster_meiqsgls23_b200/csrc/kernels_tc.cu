@@ -1701,10 +1701,12 @@ int tc_prepare_weights(occu_ctx *ctx, cudaStream_t st) {
   if (ctx->wimg_version == ctx->params_version) return 0;
   const occu_config &c = ctx->cfg;
   const ParamLayout &L = ctx->layout;
-  // slots: 6 kinds per ANEE layer, plus "layer" L for the decoder's FFN (kinds 0, 1)
-  if (ctx->wimg.ensure(size_t(c.L + 1) * 6 * WIMG_MAX) != cudaSuccess ||
-      ctx->wfexp.ensure(size_t(c.L + 1) * 6 * 2 * sizeof(int)) != cudaSuccess ||
-      ctx->wjobs.ensure(size_t(c.L + 1) * 6 * sizeof(WImageJob)) != cudaSuccess)
+  // slots: 6 kinds per ANEE layer, plus "layer" L for the decoder's FFN (kinds 0, 1) and
+  // "layer" L + 1 + j for Graphormer layer j (kinds 0-5: W_q, W_k, W_v, W_o, FFN W1, W2)
+  const size_t nslot = size_t(c.L + 1 + c.graphormer) * 6;
+  if (ctx->wimg.ensure(nslot * WIMG_MAX) != cudaSuccess ||
+      ctx->wfexp.ensure(nslot * 2 * sizeof(int)) != cudaSuccess ||
+      ctx->wjobs.ensure(nslot * sizeof(WImageJob)) != cudaSuccess)
     return -int(cudaErrorMemoryAllocation);
   std::vector<WImageJob> jobs;
   const float *P = ctx->params.as<float>();
@@ -1738,6 +1740,17 @@ int tc_prepare_weights(occu_ctx *ctx, cudaStream_t st) {
     };
     addd(0, P + L.D.P.W1);
     addd(1, P + L.D.P.W2);
+  }
+  for (int j = 0; j < c.graphormer; ++j) {      // NEXT-3 Graphormer: six d x d matrices
+    const GphOff &g = L.G[j];
+    const size_t ws[6] = {g.Wq, g.Wk, g.Wv, g.Wo, g.F.W1, g.F.W2};
+    for (int kind = 0; kind < 6; ++kind) {
+      WImageJob jb;
+      jb.W = P + ws[kind]; jb.D = c.d; jb.K = c.d; jb.transW = 0; jb.bf16 = 0;
+      jb.img = const_cast<uint8_t *>(tc_wimg(ctx, kind, c.L + 1 + j));
+      jb.fexp = const_cast<int *>(tc_wfexp(ctx, kind, c.L + 1 + j));
+      jobs.push_back(jb);
+    }
   }
   // job table: pointers are fixed for the ctx, re-uploaded only with the images
   if (cudaMemcpyAsync(ctx->wjobs.ptr, jobs.data(), jobs.size() * sizeof(WImageJob),
@@ -1975,6 +1988,24 @@ int launch_bias_tc(const occu_ctx *ctx, const float *A, int K, int R, int wkind,
   if (R <= 0) return 0;
   return ctx->cfg.d == 64 ? bias_impl<64>(ctx, A, K, R, wkind, layer, bias, relu, out, name, st)
                           : bias_impl<128>(ctx, A, K, R, wkind, layer, bias, relu, out, name, st);
+}
+template <int D>
+static int bias_add_impl(const occu_ctx *ctx, const float *A, int K, int R, int wkind, int layer,
+                         const float *bias, const float *add, float *out, const char *name,
+                         cudaStream_t st) {
+  RowGemmArgs r{};
+  r.slope = ctx->cfg.slope;
+  r.A = A; r.K = K; r.R = R; r.out = out; r.bias = bias; r.add = add;
+  r.wimg = tc_wimg(ctx, wkind, layer); r.wfexp = tc_wfexp(ctx, wkind, layer);
+  return launch_rowgemm<D, EPI_PLAIN>(ctx, r, name, st);
+}
+// out = A·Wᵀ + bias + add (residual), rows R (Graphormer output projections)
+int launch_bias_add_tc(const occu_ctx *ctx, const float *A, int K, int R, int wkind, int layer,
+                       const float *bias, const float *add, float *out, const char *name,
+                       cudaStream_t st) {
+  if (R <= 0) return 0;
+  return ctx->cfg.d == 64 ? bias_add_impl<64>(ctx, A, K, R, wkind, layer, bias, add, out, name, st)
+                          : bias_add_impl<128>(ctx, A, K, R, wkind, layer, bias, add, out, name, st);
 }
 int launch_bwd_edge_tc(const occu_ctx *ctx, const DevCsr &csr, int layer, const float *e_in, int Ke,
                        const float *e, const float *de, const float *p, const float *q, float *DZ,

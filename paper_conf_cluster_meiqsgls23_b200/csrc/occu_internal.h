@@ -24,6 +24,8 @@ const char *global_error();
 struct FfnOff { size_t W1, b1, W2, b2; };
 struct MabOff { size_t Wq, bq, Wk, bk, Wv, bv, Wo, bo, ln1_g, ln1_b; FfnOff F; size_t ln2_g, ln2_b; };
 struct DecLayout { size_t S; FfnOff P; MabOff M1, M2; FfnOff D; };
+// Graphormer layer (NEXT-3): ln1, MHA (Wq bq Wk bk Wv bv Wo bo), ln2, FFN.
+struct GphOff { size_t ln1_g, ln1_b, Wq, bq, Wk, bk, Wv, bv, Wo, bo, ln2_g, ln2_b; FfnOff F; };
 
 struct ParamLayout {
   // offsets (in floats) of each tensor inside the flat parameter vector
@@ -32,6 +34,7 @@ struct ParamLayout {
   std::vector<int> d_in, de_in;
   bool dec = false;
   DecLayout D{};
+  std::vector<GphOff> G;    // Graphormer layers
   int head_in = 0;          // W_1 columns: d (mean readout) or k·d (decoder)
 };
 ParamLayout make_layout(const occu_config &c);
@@ -63,6 +66,8 @@ struct Workspace {
   DevBuf anf[2], aef[2], acsr[2];   // occu_predict_async: double-buffered input staging
   DevBuf dT, dZ;           // decoder readout: per-node FFN hidden / output rows [N][d]
   DevBuf dprep;            // decoder readout: folded key map M [d][16] and offsets c [16]
+  std::vector<DevBuf> gh;  // Graphormer layer outputs [N][d] (per layer)
+  DevBuf gx, gqkv, go;     // Graphormer scratch: LN output [N][d], Q|K|V [3][N][d], attention [N][d]
   void release_all();
 };
 
@@ -227,6 +232,11 @@ int launch_readout_head(const occu_ctx *ctx, const DevCsr &csr, const float *h, 
 // NEXT-2 readout (kernels_decoder.cu): Z = FFN(h_L) on tensor cores (T = ReLU(h W1ᵀ + b1),
 // Z = T W2ᵀ + b2), then per graph the k-seed attention pool over Z, the MAB / SAB / FFN tail
 // and the head; r receives the flattened decoder output [B][k·d].
+int launch_graphormer_layer(const occu_ctx *ctx, const DevCsr &csr, int j, const float *h_in,
+                            float *h_out, float *X, float *QKV, float *O, cudaStream_t st);
+int launch_bias_add_tc(const occu_ctx *ctx, const float *A, int K, int R, int wkind, int layer,
+                       const float *bias, const float *add, float *out, const char *name,
+                       cudaStream_t st);
 int launch_set_decoder(const occu_ctx *ctx, const DevCsr &csr, const float *hL, float *T, float *Z,
                        float *r, float *c, float *yhat, cudaStream_t st);
 // Row-GEMM out = act(A Wᵀ + bias) over R rows on tensor cores with a prebuilt image (kernels_tc.cu).

@@ -47,9 +47,9 @@ void Workspace::release_all() {
   DevBuf *bufs[] = {&node_feat, &edge_feat, &targets, &out_occ, &csr, &e0, &g, &r, &c, &yhat,
                     &dy, &dc, &dr, &dh, &dhprev, &dP, &MG, &DV, &DZ, &deA, &deB, &dalpha,
                     &dpq, &partial, &loss, &tcpart, &dpart, &rpart, &anf[0], &anf[1],
-                    &aef[0], &aef[1], &acsr[0], &acsr[1], &dT, &dZ, &dprep};
+                    &aef[0], &aef[1], &acsr[0], &acsr[1], &dT, &dZ, &dprep, &gx, &gqkv, &go};
   for (DevBuf *b : bufs) b->release();
-  for (auto *v : {&hbar, &p, &q, &e, &h, &gs})
+  for (auto *v : {&hbar, &p, &q, &e, &h, &gs, &gh})
     for (DevBuf &b : *v) b.release();
 }
 
@@ -172,6 +172,15 @@ occu_status validate_cfg(const occu_config *c) {
         c->k * c->heads > 16 || c->d % c->heads)
       return fail(nullptr, OCCU_EINVAL, "decoder: k in [1,8], heads in {1,2,4,8}, k*heads <= 16");
   }
+  if (c->graphormer < 0 || c->graphormer > 4)
+    return fail(nullptr, OCCU_EINVAL, "graphormer must be in [0, 4]");
+  if (c->graphormer > 0) {
+    if (c->prec != OCCU_FP32 || c->F_n > 128)
+      return fail(nullptr, OCCU_EINVAL, "Graphormer layers run in OCCU_FP32 on the tensor-core path");
+    if (c->heads < 1 || c->d % c->heads ||
+        !(c->d / c->heads == 16 || c->d / c->heads == 32 || c->d / c->heads == 64))
+      return fail(nullptr, OCCU_EINVAL, "Graphormer: d / heads must be 16, 32 or 64");
+  }
   return OCCU_OK;
 }
 
@@ -251,7 +260,8 @@ occu_status forward(occu_ctx *ctx, const DevCsr &csr, const float *nf, const flo
   // and the readout's node sums folded into the last aggregation (chunk partials).
   const bool fuse_e0 = tc && c.F_e <= 16;
   const bool dec = c.readout == OCCU_READOUT_SET_DECODER;
-  const bool fuse_ro = tc && (bf || ctx->path == 0) && !dec;
+  const bool gph = c.graphormer > 0;
+  const bool fuse_ro = tc && (bf || ctx->path == 0) && !dec && !gph;
   if (!fuse_e0) LK(launch_permute_rows(ctx, ef, csr.in_eid, csr.E, c.F_e, w.e0.as<float>(), s), "permute e0");
   if (tc) LK(tc_prepare_weights(ctx, s), "weight images");
   float *rpart = nullptr;
@@ -300,16 +310,32 @@ occu_status forward(occu_ctx *ctx, const DevCsr &csr, const float *nf, const flo
       LK(launch_forward_layer(ctx, csr, a, s), "forward layer");
     }
   }
+  const float *h_top = w.h[c.L - 1].as<float>();
+  if (gph) {
+    // NEXT-3: Graphormer layers over each graph's node set (ping-pong between two buffers)
+    if (w.gh.size() < size_t(c.graphormer)) w.gh.resize(c.graphormer);
+    for (int j = 0; j < c.graphormer; ++j) CK(w.gh[j].ensure(size_t(csr.N) * c.d * 4), "alloc graphormer states");
+    CK(w.gx.ensure(size_t(csr.N) * c.d * 4), "alloc graphormer scratch");
+    CK(w.gqkv.ensure(size_t(csr.N) * 3 * c.d * 4), "alloc graphormer scratch");
+    CK(w.go.ensure(size_t(csr.N) * c.d * 4), "alloc graphormer scratch");
+    for (int j = 0; j < c.graphormer; ++j) {
+      float *out = w.gh[j].as<float>();
+      LK(launch_graphormer_layer(ctx, csr, j, h_top, out, w.gx.as<float>(), w.gqkv.as<float>(),
+                                 w.go.as<float>(), s),
+         "graphormer layer");
+      h_top = out;
+    }
+  }
   if (dec) {
     // NEXT-2: Set-Transformer decoder per graph, head on the flattened k·d output
     CK(w.dT.ensure(size_t(csr.N) * c.d * 4), "alloc decoder scratch");
     CK(w.dZ.ensure(size_t(csr.N) * c.d * 4), "alloc decoder scratch");
     CK(w.r.ensure(size_t(csr.B) * c.k * c.d * 4), "alloc r");
-    LK(launch_set_decoder(ctx, csr, w.h[c.L - 1].as<float>(), w.dT.as<float>(), w.dZ.as<float>(),
+    LK(launch_set_decoder(ctx, csr, h_top, w.dT.as<float>(), w.dZ.as<float>(),
                           w.r.as<float>(), w.c.as<float>(), w.yhat.as<float>(), s),
        "set decoder");
   } else {
-    LK(launch_readout_head(ctx, csr, fuse_ro ? rpart : w.h[c.L - 1].as<float>(), fuse_ro, P,
+    LK(launch_readout_head(ctx, csr, fuse_ro ? rpart : h_top, fuse_ro, P,
                            w.r.as<float>(), w.c.as<float>(), w.yhat.as<float>(), s),
        "readout/head");
   }
@@ -368,6 +394,8 @@ occu_status grads_impl(occu_ctx *ctx, const occu_batch *batch, const float *targ
     return fail(ctx, OCCU_EINVAL, "global_num_graphs < local num_graphs");
   if (ctx->cfg.readout == OCCU_READOUT_SET_DECODER)
     return fail(ctx, OCCU_EINVAL, "the Set-Transformer decoder readout is inference-only in this build");
+  if (ctx->cfg.graphormer > 0)
+    return fail(ctx, OCCU_EINVAL, "Graphormer layers are inference-only in this build");
   ctx->launches = 0;
   if ((st = resolve_csr(ctx, batch->csr, csr)) != OCCU_OK) return st;
   if ((st = stage_inputs(ctx, csr, batch->node_feat, batch->edge_feat, targets, stg)) != OCCU_OK)
@@ -799,6 +827,8 @@ occu_status occu_set_kernel_path(occu_ctx *ctx, int path) {
     return fail(ctx, OCCU_EINVAL, "reading B (NEIGHBOR_SOFTMAX) runs on kernel path 0 only");
   if (ctx->cfg.readout == OCCU_READOUT_SET_DECODER && path != 0)
     return fail(ctx, OCCU_EINVAL, "the decoder readout runs on kernel path 0 only");
+  if (ctx->cfg.graphormer > 0 && path != 0)
+    return fail(ctx, OCCU_EINVAL, "Graphormer layers run on kernel path 0 only");
   ctx->path = path;
   return OCCU_OK;
 }
@@ -816,6 +846,8 @@ occu_status occu_get_tensor(occu_ctx *ctx, int32_t which, int32_t layer, void *h
   const int d = ctx->cfg.d;
   const bool per_layer = which <= OCCU_T_H;
   if (per_layer && (layer < 0 || layer >= ctx->cfg.L)) return fail(ctx, OCCU_EINVAL, "bad layer");
+  if (which == OCCU_T_GPH && (layer < 0 || layer >= ctx->cfg.graphormer))
+    return fail(ctx, OCCU_EINVAL, "bad Graphormer layer");
   const void *src = nullptr;
   size_t need = 0;
   Workspace &w = ctx->ws;
@@ -833,6 +865,7 @@ occu_status occu_get_tensor(occu_ctx *ctx, int32_t which, int32_t layer, void *h
       src = w.h[layer].ptr; need = size_t(c.N) * d * 4; break;
     case OCCU_T_R: src = w.r.ptr; need = size_t(c.B) * ctx->layout.head_in * 4; break;   // [B][d] or [B][k·d]
     case OCCU_T_YHAT: src = w.yhat.ptr; need = size_t(c.B) * 4; break;
+    case OCCU_T_GPH: src = w.gh[layer].ptr; need = size_t(c.N) * d * 4; break;
     default: return fail(ctx, OCCU_EINVAL, "unknown tensor");
   }
   if (bytes != need) return fail(ctx, OCCU_EINVAL, "byte count mismatch");

@@ -3,7 +3,8 @@
 //
 // Layout, per ANEE layer i (P141-P149 with readings R1, R5):
 //   W_u[d][d_in]  W_e[d][d_e,in]  W_m[d][d]  a_s[d]  a_d[d]
-// then the head (P125, R12): W_1[d_h][d]  b_1[d_h]  w_2[d_h]  b_2[1].
+// then the Graphormer layers (NEXT-3), the decoder (NEXT-2) when configured, and the head
+// (P125, R12): W_1[d_h][d or k·d]  b_1[d_h]  w_2[d_h]  b_2[1].
 #include <math.h>
 #include <stdio.h>
 #include <string.h>
@@ -29,12 +30,23 @@ ParamLayout make_layout(const occu_config &c) {
     L.a_d.push_back(off); off += c.d;
   }
   L.head_in = c.d;
+  const size_t d = size_t(c.d), dd = d * d;
+  auto ffn = [&](FfnOff &f) {
+    f.W1 = off; off += dd; f.b1 = off; off += d; f.W2 = off; off += dd; f.b2 = off; off += d;
+  };
+  for (int j = 0; j < c.graphormer; ++j) {     // Graphormer layers (NEXT-3), file order
+    GphOff g;
+    g.ln1_g = off; off += d; g.ln1_b = off; off += d;
+    g.Wq = off; off += dd; g.bq = off; off += d;
+    g.Wk = off; off += dd; g.bk = off; off += d;
+    g.Wv = off; off += dd; g.bv = off; off += d;
+    g.Wo = off; off += dd; g.bo = off; off += d;
+    g.ln2_g = off; off += d; g.ln2_b = off; off += d;
+    ffn(g.F);
+    L.G.push_back(g);
+  }
   if (c.readout == OCCU_READOUT_SET_DECODER) {
-    const size_t d = size_t(c.d), dd = d * d;
     L.dec = true;
-    auto ffn = [&](FfnOff &f) {
-      f.W1 = off; off += dd; f.b1 = off; off += d; f.W2 = off; off += dd; f.b2 = off; off += d;
-    };
     L.D.S = off; off += size_t(c.k) * d;
     ffn(L.D.P);
     for (MabOff *m : {&L.D.M1, &L.D.M2}) {
@@ -77,13 +89,22 @@ void init_flat(const occu_config &c, uint64_t seed, std::vector<float> &out) {
     ts.push_back({L.a_s[i], size_t(c.d), 2 * c.d});
     ts.push_back({L.a_d[i], size_t(c.d), 2 * c.d});
   }
+  // fan_in -1: constant 1 (LayerNorm gain), 0: constant 0 (LayerNorm bias)
+  const size_t d = size_t(c.d), dd = d * d;
+  auto ffn = [&](const FfnOff &f) {
+    ts.push_back({f.W1, dd, c.d}); ts.push_back({f.b1, d, c.d});
+    ts.push_back({f.W2, dd, c.d}); ts.push_back({f.b2, d, c.d});
+  };
+  for (const GphOff &g : L.G) {
+    ts.push_back({g.ln1_g, d, -1}); ts.push_back({g.ln1_b, d, 0});
+    for (size_t w : {g.Wq, g.Wk, g.Wv, g.Wo}) {
+      ts.push_back({w, dd, c.d});
+      ts.push_back({w + dd, d, c.d});            // its bias follows it
+    }
+    ts.push_back({g.ln2_g, d, -1}); ts.push_back({g.ln2_b, d, 0});
+    ffn(g.F);
+  }
   if (L.dec) {
-    // fan_in -1: constant 1 (LayerNorm gain), 0: constant 0 (LayerNorm bias)
-    const size_t d = size_t(c.d), dd = d * d;
-    auto ffn = [&](const FfnOff &f) {
-      ts.push_back({f.W1, dd, c.d}); ts.push_back({f.b1, d, c.d});
-      ts.push_back({f.W2, dd, c.d}); ts.push_back({f.b2, d, c.d});
-    };
     ts.push_back({L.D.S, size_t(c.k) * d, c.d});
     ffn(L.D.P);
     for (const MabOff *m : {&L.D.M1, &L.D.M2}) {
@@ -125,6 +146,12 @@ uint64_t fnv1a64(const void *data, size_t n) {
   return h;
 }
 
+// File version: 1 = mean readout, 2 = decoder readout (+ u32 readout, k, heads), 3 = with
+// Graphormer layers (+ u32 readout, k, heads, graphormer).
+static uint32_t file_version(const occu_config &c) {
+  return c.graphormer > 0 ? 3u : c.readout == OCCU_READOUT_SET_DECODER ? 2u : 1u;
+}
+
 // header: "OCCUW001", u32 version, L, F_n, F_e, d, d_h, aggr, msg, f32 slope
 bool write_file(const char *path, const char magic[8], const occu_config &c,
                 const std::vector<std::pair<const void *, size_t>> &chunks, std::string &err) {
@@ -133,12 +160,13 @@ bool write_file(const char *path, const char magic[8], const occu_config &c,
     err = std::string("cannot open ") + path + " for writing";
     return false;
   }
-  const bool v2 = c.readout == OCCU_READOUT_SET_DECODER;
-  uint32_t hdr[8] = {v2 ? 2u : 1u, uint32_t(c.L), uint32_t(c.F_n), uint32_t(c.F_e), uint32_t(c.d),
+  const uint32_t ver = file_version(c);
+  const size_t next = ver == 3 ? 4 : ver == 2 ? 3 : 0;
+  uint32_t hdr[8] = {ver, uint32_t(c.L), uint32_t(c.F_n), uint32_t(c.F_e), uint32_t(c.d),
                      uint32_t(c.d_h), uint32_t(c.aggr), uint32_t(c.msg)};
-  const uint32_t ext[3] = {uint32_t(c.readout), uint32_t(c.k), uint32_t(c.heads)};
+  const uint32_t ext[4] = {uint32_t(c.readout), uint32_t(c.k), uint32_t(c.heads), uint32_t(c.graphormer)};
   bool ok = fwrite(magic, 1, 8, f) == 8 && fwrite(hdr, 4, 8, f) == 8 &&
-            fwrite(&c.slope, 4, 1, f) == 1 && (!v2 || fwrite(ext, 4, 3, f) == 3);
+            fwrite(&c.slope, 4, 1, f) == 1 && fwrite(ext, 4, next, f) == next;
   uint64_t h = 0xCBF29CE484222325ull;
   for (auto &ch : chunks) {
     ok = ok && fwrite(ch.first, 1, ch.second, f) == ch.second;
@@ -167,21 +195,23 @@ occu_status read_file(const char *path, const char magic[8], const occu_config &
   size_t n;
   while ((n = fread(buf, 1, sizeof buf, f)) > 0) raw.insert(raw.end(), buf, buf + n);
   fclose(f);
-  const bool v2 = c.readout == OCCU_READOUT_SET_DECODER;
-  const size_t hdr = 8 + 32 + 4 + (v2 ? 12 : 0);
+  const uint32_t ver = file_version(c);
+  const size_t next = ver == 3 ? 4 : ver == 2 ? 3 : 0;
+  const size_t hdr = 8 + 32 + 4 + 4 * next;
   if (raw.size() < hdr + 8 || memcmp(raw.data(), magic, 8) != 0) {
     err = "bad magic or truncated file";
     return OCCU_EFORMAT;
   }
-  uint32_t h[8], ext[3] = {0, 0, 0};
+  uint32_t h[8], ext[4] = {0, 0, 0, 0};
   memcpy(h, raw.data() + 8, 32);
   float slope;
   memcpy(&slope, raw.data() + 40, 4);
-  if (v2) memcpy(ext, raw.data() + 44, 12);
-  if (h[0] != (v2 ? 2u : 1u) || int(h[1]) != c.L || int(h[2]) != c.F_n || int(h[3]) != c.F_e ||
+  memcpy(ext, raw.data() + 44, 4 * next);
+  if (h[0] != ver || int(h[1]) != c.L || int(h[2]) != c.F_n || int(h[3]) != c.F_e ||
       int(h[4]) != c.d || int(h[5]) != c.d_h || int(h[6]) != c.aggr || int(h[7]) != c.msg ||
       slope != c.slope ||
-      (v2 && (int(ext[0]) != c.readout || int(ext[1]) != c.k || int(ext[2]) != c.heads))) {
+      (next >= 3 && (int(ext[0]) != c.readout || int(ext[1]) != c.k || int(ext[2]) != c.heads)) ||
+      (next == 4 && int(ext[3]) != c.graphormer)) {
     err = "file config does not match the context config";
     return OCCU_EINVAL;
   }

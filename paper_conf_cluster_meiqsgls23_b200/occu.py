@@ -20,7 +20,7 @@ OCCU_OK, OCCU_EINVAL, OCCU_ENOMEM, OCCU_ECUDA, OCCU_EFORMAT, OCCU_ENOTREADY, OCC
 AGGR_SUM, AGGR_MEAN = 0, 1
 MSG_CHANNEL_SOFTMAX, MSG_NEIGHBOR_SOFTMAX = 0, 1
 FP32, BF16 = 0, 1
-T_HBAR, T_P, T_Q, T_E, T_H, T_R, T_YHAT = range(7)
+T_HBAR, T_P, T_Q, T_E, T_H, T_R, T_YHAT, T_GPH = range(8)
 STATUS_NAMES = {0: "OK", 1: "EINVAL", 2: "ENOMEM", 3: "ECUDA", 4: "EFORMAT", 5: "ENOTREADY",
                 6: "ENCCL"}
 
@@ -45,7 +45,7 @@ class Config(C.Structure):
     _fields_ = [("L", C.c_int32), ("F_n", C.c_int32), ("F_e", C.c_int32), ("d", C.c_int32),
                 ("d_h", C.c_int32), ("aggr", C.c_int32), ("msg", C.c_int32), ("prec", C.c_int32),
                 ("slope", C.c_float), ("readout", C.c_int32), ("k", C.c_int32),
-                ("heads", C.c_int32)]
+                ("heads", C.c_int32), ("graphormer", C.c_int32)]
 
 
 class GraphView(C.Structure):
@@ -144,9 +144,9 @@ READOUT_MEAN, READOUT_SET_DECODER = 0, 1
 
 
 def config(L=3, F_n=80, F_e=4, d=128, d_h=None, aggr=AGGR_SUM, msg=MSG_CHANNEL_SOFTMAX,
-           prec=FP32, slope=0.01, readout=READOUT_MEAN, k=4, heads=4):
+           prec=FP32, slope=0.01, readout=READOUT_MEAN, k=4, heads=4, graphormer=0):
     return Config(L, F_n, F_e, d, d if d_h is None else d_h, aggr, msg, prec, slope, readout,
-                  k if readout else 0, heads if readout else 0)
+                  k if readout else 0, heads if (readout or graphormer) else 0, graphormer)
 
 
 def num_params(cfg: Config) -> int:

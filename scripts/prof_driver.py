@@ -15,9 +15,13 @@ ap.add_argument("--path", type=int, default=0)
 ap.add_argument("--train", action="store_true")
 ap.add_argument("--graphs", type=int, default=256)
 ap.add_argument("--bf16", action="store_true")
+ap.add_argument("--graphormer", type=int, default=0)
+ap.add_argument("--decoder", action="store_true")
 a = ap.parse_args()
 dev = torch.device("cuda", 0)
-m = occu.Model(occu.config(L=3, F_n=80, F_e=4, d=128, prec=occu.BF16 if a.bf16 else occu.FP32))
+m = occu.Model(occu.config(L=3, F_n=80, F_e=4, d=128, prec=occu.BF16 if a.bf16 else occu.FP32,
+                           graphormer=a.graphormer, heads=4,
+                           readout=occu.READOUT_SET_DECODER if a.decoder else occu.READOUT_MEAN))
 m.init_weights(42)
 m.set_kernel_path(a.path)
 b = configs.cfg2(a.graphs)
