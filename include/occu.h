@@ -177,6 +177,20 @@ occu_status occu_compute_grads(occu_ctx *ctx, const occu_batch *batch, const flo
 occu_status occu_get_grads(const occu_ctx *ctx, float *host_flat, size_t n);
 occu_status occu_set_weight_decay(occu_ctx *ctx, float wd);
 
+/* ---- NEXT-4 consumer: occu-packing (P390-P392; R38) ------------------
+ * Host-side first-fit bin packing of jobs by predicted occupancy (the output of
+ * occu_predict), the paper's co-location policy: "the cumulative GPU occupancy of the DL
+ * load not exceeding 100%" (P392).  Jobs are taken in array order; job j goes to the
+ * lowest-numbered GPU slot b with load_b + occ_j <= capacity (float64, occ widened from
+ * float32, predictions < 0 counted as 0), else a new slot opens (a job larger than the
+ * capacity gets a slot of its own).  occ: host [num_jobs]; slot_of_job: host [num_jobs]
+ * (caller-allocated, written); slot_load: nullable host [num_jobs] (the first *num_slots
+ * entries are written); *num_slots = slots opened.  O(num_jobs log num_jobs).  Errors:
+ * OCCU_EINVAL for NULL pointers, num_jobs < 0, capacity not finite and > 0, or a NaN / Inf
+ * prediction (message via occu_last_error(NULL)); nothing is written then. */
+occu_status occu_pack_jobs(const float *occ, int32_t num_jobs, double capacity,
+                           int32_t *slot_of_job, double *slot_load, int32_t *num_slots);
+
 /* ---- data parallel (north_star: NCCL gradient allreduce over NVLink) ------ */
 occu_status occu_nccl_unique_id(void *out_128_bytes);
 occu_status occu_dist_init(occu_ctx *ctx, int rank, int world, const void *nccl_unique_id);

@@ -527,3 +527,28 @@ def mre(yhat, y):
 def mse(yhat, y):
     yhat, y = np.asarray(yhat, np.float64), np.asarray(y, np.float64)
     return float(np.mean((yhat - y) ** 2))
+
+
+# --------------------------------------------------------------------------
+# NEXT-4 consumer: occu-packing (P390-P392; R38).  "an appropriate packing
+# policy for multiple jobs should ensure the cumulative occupancy is at most 100%" (P390);
+# "a GPU-occupancy-based bin-packing algorithm (with co-location ensuring GPU occupancy does
+# not exceed 100%)" (P392).  Reading R38: first fit in submission order; job j goes to the
+# lowest-numbered GPU slot b with load_b + occ_j <= capacity (float64 arithmetic on the
+# float32 predictions, loads summed in placement order), else a new slot is opened;
+# predictions below 0 count as 0.  Plain O(jobs x slots) loop.
+# --------------------------------------------------------------------------
+def occu_packing(occ, capacity=1.0):
+    occ = np.maximum(np.asarray(occ, np.float32).astype(np.float64), 0.0)
+    loads = []
+    assign = np.empty(len(occ), np.int32)
+    for j, o in enumerate(occ):
+        for b, ld in enumerate(loads):
+            if ld + o <= capacity:
+                loads[b] = ld + o
+                assign[j] = b
+                break
+        else:
+            loads.append(o)
+            assign[j] = len(loads) - 1
+    return assign, np.array(loads, np.float64)

@@ -31,7 +31,7 @@ EXPORTS = [
     "occu_compute_grads", "occu_get_grads", "occu_set_weight_decay", "occu_nccl_unique_id",
     "occu_dist_init", "occu_save_state", "occu_load_state", "occu_set_keep_intermediates",
     "occu_get_tensor", "occu_last_launch_count", "occu_last_error", "occu_set_profiling",
-    "occu_profile_reset", "occu_profile_query", "occu_set_kernel_path",
+    "occu_profile_reset", "occu_profile_query", "occu_set_kernel_path", "occu_pack_jobs",
 ]
 
 
@@ -90,6 +90,7 @@ def lib():
             "occu_set_params": ([VP, VP, SZ], I32),
             "occu_get_params": ([VP, VP, SZ], I32),
             "occu_pack": ([P(GraphView), I32, P(P(CsrBatch))], I32),
+            "occu_pack_jobs": ([P(C.c_float), I32, C.c_double, P(I32), P(C.c_double), P(I32)], I32),
             "occu_batch_to_device": ([VP, P(CsrBatch), P(P(CsrBatch))], I32),
             "occu_batch_free": ([P(CsrBatch)], None),
             "occu_predict": ([VP, P(CsrBatch), VP, VP, VP], I32),
@@ -249,6 +250,20 @@ def pack_arrays(num_nodes, num_edges, src, dst) -> Csr:
     out = C.POINTER(CsrBatch)()
     _check(lib().occu_pack(views.ctypes.data_as(C.POINTER(GraphView)), n, C.byref(out)))
     return Csr(out)
+
+
+def pack_jobs(occ, capacity=1.0):
+    """occu-packing (NEXT-4, P390-P392): first-fit slots for jobs by predicted occupancy.
+    Returns (slot_of_job int32 [n], slot_load float64 [num_slots])."""
+    occ = np.ascontiguousarray(occ, dtype=np.float32)
+    n = len(occ)
+    slot = np.empty(max(n, 1), np.int32)
+    load = np.empty(max(n, 1), np.float64)
+    ns = C.c_int32(0)
+    _check(lib().occu_pack_jobs(occ.ctypes.data_as(C.POINTER(C.c_float)), n, float(capacity),
+                                slot.ctypes.data_as(C.POINTER(C.c_int32)),
+                                load.ctypes.data_as(C.POINTER(C.c_double)), C.byref(ns)))
+    return slot[:n], load[:ns.value].copy()
 
 
 def ctypes_view_ok() -> bool:

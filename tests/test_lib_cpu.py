@@ -123,3 +123,36 @@ def test_pack_arrays_matches_pack_and_oracle():
     with pytest.raises(occu.OccuError) as ei:
         occu.pack(bad)
     assert "graph 31" in str(ei.value) and "self-loop" in str(ei.value)
+
+
+# ------------------------------------------ NEXT-4: occu-packing through the C-ABI (host)
+def test_pack_jobs_matches_oracle_bit_exact():
+    rng = np.random.default_rng(11)
+    cases = [np.zeros(0, np.float32), np.array([0.3], np.float32),
+             rng.random(1000).astype(np.float32),
+             (rng.random(3000) * 0.4).astype(np.float32),            # many jobs per slot
+             np.concatenate([rng.random(200), [1.5, -0.2, 0.0, 1.0]]).astype(np.float32),
+             np.round(rng.random(500) * 8).astype(np.float32) / 8]   # exact ties at capacity
+    for occ in cases:
+        a, loads = occu.pack_jobs(occ)
+        ra, rl = oracle.occu_packing(occ)
+        assert np.array_equal(a, ra)
+        assert np.array_equal(loads, rl)
+    a, _ = occu.pack_jobs(np.full(9, 0.3, np.float32), capacity=0.6)
+    assert np.array_equal(a, oracle.occu_packing(np.full(9, 0.3, np.float32), 0.6)[0])
+
+
+def test_pack_jobs_golden_and_errors():
+    import os
+    d = {}
+    for ln in open(os.path.join(os.path.dirname(__file__), "golden", "occu_packing_first_fit.txt")):
+        if ln.strip() and not ln.startswith("#"):
+            k, *v = ln.split()
+            d[k] = v
+    a, loads = occu.pack_jobs(np.array(d["occ"], np.float32))
+    assert np.array_equal(a, np.array(d["assign"], np.int32)) and len(loads) == int(d["bins"][0])
+    for bad in (np.array([0.1, np.nan], np.float32), np.array([np.inf], np.float32)):
+        with pytest.raises(occu.OccuError):
+            occu.pack_jobs(bad)
+    with pytest.raises(occu.OccuError):
+        occu.pack_jobs(np.array([0.1], np.float32), capacity=0.0)

@@ -794,3 +794,40 @@ def test_graphormer_weights_file_v3_roundtrip(tmp_path):
     assert cf["graphormer"] == 2 and cf["readout"] == 1 and cf["k"] == 3
     assert np.array_equal(oracle.flatten(cf, p), flat.astype(np.float64))
     assert np.all(p["G1_ln2_g"] == 1.0) and np.all(p["G0_ln1_b"] == 0.0)
+
+
+# ------------------------------------------ NEXT-4: occu-packing consumer (P390-P392)
+def read_golden_packing():
+    import os
+    d = {}
+    for ln in open(os.path.join(os.path.dirname(__file__), "golden", "occu_packing_first_fit.txt")):
+        if ln.startswith("#") or not ln.strip():
+            continue
+        k, *v = ln.split()
+        d[k] = v
+    return (np.array(d["occ"], np.float32), np.array(d["assign"], np.int32), int(d["bins"][0]))
+
+
+def test_occu_packing_golden_first_fit():
+    occ, assign, bins = read_golden_packing()
+    a, loads = oracle.occu_packing(occ)
+    assert np.array_equal(a, assign) and len(loads) == bins
+
+
+def test_occu_packing_invariants_and_bounds():
+    """Every slot stays within capacity (jobs <= capacity), loads are the sums of their jobs,
+    first fit never leaves two slots at most half full (so slots <= 2*sum + 1), and the
+    count is at least ceil(sum); equal-size jobs of 1/k fill slots exactly k at a time."""
+    rng = np.random.default_rng(4)
+    for n in (1, 17, 500):
+        occ = rng.random(n).astype(np.float32)
+        a, loads = oracle.occu_packing(occ)
+        assert np.all(loads <= 1.0)
+        assert np.allclose(np.bincount(a, weights=occ.astype(np.float64)), loads, rtol=0, atol=1e-12)
+        assert np.sum(loads <= 0.5) <= 1
+        assert len(loads) >= np.ceil(occ.astype(np.float64).sum() - 1e-9)
+        assert len(loads) <= 2 * occ.astype(np.float64).sum() + 1
+    a, loads = oracle.occu_packing(np.full(12, 0.25, np.float32))
+    assert np.array_equal(a, np.repeat(np.arange(3), 4))
+    a, _ = oracle.occu_packing(np.array([-0.1, 1.3, 0.2], np.float32))   # clamp, oversize alone
+    assert np.array_equal(a, [0, 1, 0])
