@@ -261,6 +261,7 @@ def main():
     ap.add_argument("--no-train", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--no-cfg3", action="store_true", help="skip the CFG3 training line")
+    ap.add_argument("--no-extra", action="store_true", help="skip the CFG1 / CFG4 / CFG5 lines")
     ap.add_argument("--cfg3-graphs", type=int, default=512, help="CFG3 graphs per rank")
     ap.add_argument("--no-flush", action="store_true")
     ap.add_argument("--no-bf16", action="store_true", help="skip the OCCU_BF16 inference line")
@@ -689,6 +690,167 @@ def main():
             del m3
         del nf3, ef3, yt3, csr3
 
+    # ---- CFG1 (BASELINE.json configs[0]): one LeNet-5 training graph, L=2, d=64, FP32 forward;
+    # latency-bound (~12 KB of features): per-graph latency with device-resident inputs, plus the
+    # same forward replayed from a captured CUDA graph
+    cfg1 = None
+    if args.path == 0 and not args.no_extra:
+        b1 = configs.cfg1()
+        m1 = occu.Model(occu.config(L=2, F_n=80, F_e=4, d=64), device=local, stream=stream.cuda_stream)
+        m1.init_weights(42)
+        csr1 = m1.to_device(occu.pack(b1.graphs))
+        nf1 = torch.from_numpy(b1.node_feat).to(dev)
+        ef1 = torch.from_numpy(b1.edge_feat).to(dev)
+        out1 = torch.empty(1, dtype=torch.float32, device=dev)
+        f1 = lambda: m1.predict(csr1, nf1, ef1, out1)
+        reps = 1000
+        for _ in range(20):
+            f1()
+        torch.cuda.synchronize()
+        e0 = torch.cuda.Event(enable_timing=True)
+        e1 = torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        for _ in range(reps):
+            f1()
+        e1.record(stream)
+        torch.cuda.synchronize()
+        us1 = max_over_ranks(e0.elapsed_time(e1) * 1e3 / reps)
+        cfg1 = {"workload": "CFG1 (BASELINE.json configs[0]): 1 LeNet-5 training graph "
+                            "(%d nodes, %d edges), L=2, d=64, FP32 forward" % (b1.num_nodes, b1.num_edges),
+                "value": world * 1e6 / us1, "unit": "graphs/s", "us_per_graph": us1,
+                "repetitions": reps, "launches_per_forward": m1.last_launch_count(),
+                "bound": "launch latency (inputs ~12 KB: 18 ns of HBM)", "cuda_graph": None}
+        try:      # the same forward captured once and replayed (launch overhead amortised)
+            side = torch.cuda.Stream(dev)
+            m1g = occu.Model(occu.config(L=2, F_n=80, F_e=4, d=64), device=local, stream=side.cuda_stream)
+            m1g.init_weights(42)
+            out1g = torch.empty(1, dtype=torch.float32, device=dev)
+            with torch.cuda.stream(side):
+                for _ in range(3):
+                    m1g.predict(csr1, nf1, ef1, out1g)
+            torch.cuda.synchronize()
+            cg = torch.cuda.CUDAGraph()
+            with torch.cuda.graph(cg, stream=side):
+                m1g.predict(csr1, nf1, ef1, out1g)
+            torch.cuda.synchronize()
+            cg.replay()
+            torch.cuda.synchronize()
+            assert torch.equal(out1g, out1), "graph replay differs from the eager forward"
+            for _ in range(20):
+                cg.replay()
+            torch.cuda.synchronize()
+            e0.record(stream)
+            for _ in range(reps):
+                cg.replay()
+            e1.record(stream)
+            torch.cuda.synchronize()
+            usg = max_over_ranks(e0.elapsed_time(e1) * 1e3 / reps)
+            cfg1["cuda_graph"] = {"value": world * 1e6 / usg, "unit": "graphs/s", "us_per_graph": usg}
+            del cg, m1g
+        except Exception as ex:                       # noqa: BLE001 — reported, not hidden
+            cfg1["cuda_graph"] = {"unavailable": str(ex)[:200]}
+        del m1
+
+    # ---- CFG4 / CFG5 (BASELINE.json configs[3], configs[4]): the 20-family mixture.  Every
+    # rank generates its own contiguous shard (seeded by graph index): CFG4 = data-parallel
+    # training on 256-graph micro-batches per rank (epoch of 50,000 graphs extrapolated from
+    # the timed steps); CFG5 = graph-sharded inference in launch batches of 1,024 graphs (<=
+    # 4,096) with no collective, 1M graphs extrapolated, then the occu-packing consumer.
+    cfg4 = cfg5 = None
+    if args.path == 0 and not args.no_extra:
+        mb4 = [configs.mixture(256, 1004, start=(k * world + rank) * 256) for k in range(2)]
+        dev4 = []
+        for bb in mb4:
+            dev4.append((model.to_device(occu.pack(bb.graphs)), torch.from_numpy(bb.node_feat).to(dev),
+                         torch.from_numpy(bb.edge_feat).to(dev), torch.from_numpy(bb.targets).to(dev)))
+        gB4 = 256 * world
+        m4_trained = None
+        wc4 = weights.ModelConfig(L=3, F_n=80, F_e=4, d=128, d_h=128)
+        unit_flat = weights.unit_scale(wc4, weights.init_flat(wc4, 42))
+        for prec, key in ((occu.FP32, "f32"), (occu.BF16, "bf16")):
+            m4 = occu.Model(occu.config(L=3, F_n=80, F_e=4, d=128, prec=prec), device=local,
+                            stream=stream.cuda_stream)
+            m4.set_params(unit_flat)          # unit-scale weights (R22): ŷ varies per graph
+            if pg and world > 1:
+                uid = [occu.Model.nccl_unique_id() if rank == 0 else None]
+                pg.broadcast_object_list(uid, src=0)
+                m4.dist_init(rank, world, uid[0])
+            it = [0]
+
+            def st4():
+                c_, n_, e_, y_ = dev4[it[0] % len(dev4)]
+                it[0] += 1
+                m4.train_step(c_, n_, e_, y_, 1e-3, global_num_graphs=gB4, want_loss=False)
+            timed(st4, args.warmup, mdl=m4)
+            bar()
+            t4, l4 = timed(st4, args.steps, mdl=m4)
+            bar()
+            ms4 = max_over_ranks(float(np.sum(t4)) / args.steps)
+            steps_epoch = -(-50000 // gB4)
+            ent = {"value": gB4 / (ms4 * 1e-3), "unit": "graphs/s", "ms_per_step": ms4,
+                   "dtype": key, "gpu_launches": l4, "steps_per_epoch": steps_epoch,
+                   "epoch_s_extrapolated": steps_epoch * ms4 * 1e-3}
+            if cfg4 is None:
+                cfg4 = {"workload": "CFG4 (BASELINE.json configs[3]): 20-family mixture, 256-graph "
+                                    "micro-batch per rank, global batch 256 x %d, epoch of 50,000 graphs" % world,
+                        "nodes_per_microbatch": [bb.num_nodes for bb in mb4],
+                        "edges_per_microbatch": [bb.num_edges for bb in mb4],
+                        "includes": "forward with saves, MSE, backward, "
+                                    + ("NCCL allreduce, " if world > 1 else "") + "Adam",
+                        "sharding": "contiguous per-rank shards of the seeded mixture"}
+            c_, n_, e_, y_ = dev4[0]
+            ent["loss_after"] = m4.train_step(c_, n_, e_, y_, 1e-3, global_num_graphs=gB4)
+            cfg4[key] = ent
+            m4_trained = m4
+        # CFG5: inference on 1,024-graph launch batches (2 CFG4 shards + 2 more per rank)
+        mb5 = mb4 + [configs.mixture(256, 1004, start=(k * world + rank) * 256) for k in range(2, 4)]
+        g5 = [g_ for bb in mb5 for g_ in bb.graphs]
+        nf5 = torch.from_numpy(np.concatenate([bb.node_feat for bb in mb5])).to(dev)
+        ef5 = torch.from_numpy(np.concatenate([bb.edge_feat for bb in mb5])).to(dev)
+        B5 = len(g5)
+        csr5 = model.to_device(occu.pack(g5))
+        cfg5 = {"workload": "CFG5 (BASELINE.json configs[4]): 20-family mixture, graph-sharded "
+                            "inference, launch batches of %d graphs per GPU, no collective" % B5,
+                "nodes_per_batch": int(nf5.shape[0]), "edges_per_batch": int(ef5.shape[0])}
+        for prec, key in ((occu.BF16, "bf16"), (occu.FP32, "f32")):
+            m5 = occu.Model(occu.config(L=3, F_n=80, F_e=4, d=128, prec=prec), device=local,
+                            stream=stream.cuda_stream)
+            m5.set_params(unit_flat)
+            out5 = torch.empty(B5, dtype=torch.float32, device=dev)
+            f5 = lambda: m5.predict(csr5, nf5, ef5, out5)
+            timed(f5, args.warmup, mdl=m5)
+            bar()
+            t5, l5 = timed(f5, args.steps, mdl=m5)
+            bar()
+            ms5 = max_over_ranks(float(np.sum(t5)) / args.steps)
+            v5 = B5 * world / (ms5 * 1e-3)
+            cfg5[key] = {"value": v5, "unit": "graphs/s", "ms_per_batch": ms5, "dtype": key,
+                         "gpu_launches": l5, "one_million_graphs_s_extrapolated": 1e6 / v5}
+            del m5
+        # the CFG4-trained BF16 model predicts the CFG5 batch; those predictions are packed
+        out5 = torch.empty(B5, dtype=torch.float32, device=dev)
+        m4_trained.predict(csr5, nf5, ef5, out5)
+        occ = out5.cpu().numpy()
+        del m4_trained
+        # occu-packing consumer (NEXT-4, P390-P392) on the predictions, and on 1M of them
+        occ_m = np.resize(occ, 1_000_000).astype(np.float32)
+        t0p = time.perf_counter()
+        slots, loads = occu.pack_jobs(occ_m)
+        tp = time.perf_counter() - t0p
+        tgt = np.resize(np.concatenate([bb.targets for bb in mb5]), 1_000_000).astype(np.float32)
+        _, tloads = occu.pack_jobs(tgt)
+        cfg5["occu_packing"] = {"jobs": int(len(occ_m)), "slots": int(len(loads)),
+                                "slots_by_synthetic_labels": int(len(tloads)),
+                                "mean_label_occupancy": float(np.mean(tgt)),
+                                "mean_predicted_occupancy": float(np.mean(occ)),
+                                "predicted_occupancy_p10_p90": [float(np.percentile(occ, 10)),
+                                                                float(np.percentile(occ, 90))],
+                                "host_ms": tp * 1e3, "mean_slot_occupancy": float(loads.mean()),
+                                "what": "first-fit slots, cumulative predicted occupancy <= 1.0 "
+                                        "(host C++, occu_pack_jobs); predictions of the CFG4-trained BF16 model on the "
+                                        "CFG5 batch, tiled to 1M jobs"}
+        del nf5, ef5, csr5, dev4
+
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu:
         cpu = cpu_baseline_sample()
@@ -720,6 +882,9 @@ def main():
             "graphormer": graphormer,
             "train": train,
             "train_cfg3": train_cfg3,
+            "cfg1": cfg1,
+            "cfg4_train": cfg4,
+            "cfg5_infer": cfg5,
             "cpu_baseline": cpu,
         }
         print(json.dumps(line), flush=True)
