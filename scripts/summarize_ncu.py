@@ -2,7 +2,7 @@
 import csv, io, json, os, re, subprocess, sys, collections
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 tag = sys.argv[1] if len(sys.argv) > 1 else "r01"
-out = os.path.join(ROOT, "profiles")
+out = os.environ.get("PROFILES_OUT", os.path.join(ROOT, "profiles"))
 os.makedirs(out, exist_ok=True)
 
 def kname(full):
@@ -10,7 +10,9 @@ def kname(full):
     if m:
         return ["node_tc", "edge_tc", "gate_tc", "plain_tc", "gatebwd_tc", "edgebwd_tc",
                 "gateagg_tc"][int(m.group(2))]
-    for k, v in [("edgegate", "edge_gate_tc"), ("edge_small", "edge_small"), ("wgrad_tc", "wgrad_tc"), ("wimage", "wimage"),
+    for k, v in [("gph_attn", "gph_attn"), ("gph_ln", "gph_ln"), ("set_decoder_prep", "set_decoder_prep"),
+                 ("set_decoder_kernel", "set_decoder"), ("gather_segsoftmax", "gather_segsoftmax"),
+                 ("edgegate", "edge_gate_tc"), ("edge_small", "edge_small"), ("wgrad_tc", "wgrad_tc"), ("wimage", "wimage"),
                  ("split_reduce", "split_reduce"), ("agg_fixup", "agg_fixup"),
                  ("wgrad_skinny", "wgrad_skinny"), ("gather_segsum", "gather_segsum"),
                  ("readout_head", "readout_head"), ("permute_rows", "permute_e0"),
@@ -94,11 +96,15 @@ def capture(reps):
 traffic = capture((("prof_full", "scripts/prof_driver.py (CFG2 inference)"),
                    ("prof_train", "scripts/prof_driver.py --train (CFG2 training)")))
 traffic_bf = capture((("prof_bf16", "scripts/prof_driver.py --bf16 (CFG2 inference, OCCU_BF16)"),))
+traffic_nx = capture((("prof_next", "scripts/prof_driver.py --graphormer 2 --decoder (CFG2 inference, NEXT-2/3)"),))
+if traffic_nx:
+    json.dump(traffic_nx, open(os.path.join(out, "traffic_next.json"), "w"), indent=1)
 json.dump(traffic, open(os.path.join(out, "traffic.json"), "w"), indent=1)
 if traffic_bf:
     json.dump(traffic_bf, open(os.path.join(out, "traffic_bf16.json"), "w"), indent=1)
 with open(os.path.join(out, f"{tag}_ncu_summary.md"), "w") as f:
-  for title, traffic in (("OCCU_FP32 (inference + training)", traffic), ("OCCU_BF16 inference", traffic_bf)):
+  for title, traffic in (("OCCU_FP32 (inference + training)", traffic), ("OCCU_BF16 inference", traffic_bf),
+                         ("NEXT-2/3 kernels: Graphormer x2 + decoder readout, OCCU_FP32 inference", traffic_nx)):
     if not traffic:
         continue
     f.write(f"# {tag}: ncu --set full --clock-control none (serialised, cold-cache replays), {title}\n\n")
