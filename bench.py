@@ -473,7 +473,9 @@ def main():
         msd = max_over_ranks(float(np.sum(td_)) / args.steps)
         algd = algorithmic_bytes(N, E, B, d)                  # h_L stored: unfused gather
         algd["dec_ffn_tc"] = 2 * (4 * N * d + 4 * N * d)       # T = FFN1(h_L), Z = FFN2(T)
-        algd["set_decoder"] = 4 * N * d + 4 * (B + 1) + 4 * B * (4 * d + 130)
+        parts = 4 * B * 8 * (16 * d + 32)                     # pool partials [B][8][16d + 32]
+        algd["set_decoder_pool"] = 4 * N * d + 4 * (B + 1) + parts
+        algd["set_decoder"] = parts + 4 * B * (4 * d + 130)
         kd, roofd = kernel_table(md.profile(), algd, {})
         decoder = {"value": B * world / (msd * 1e-3), "unit": "graphs/s", "ms_per_step": msd,
                    "dtype": "f32", "gpu_launches": ld_, "roofline": roofd,

@@ -37,7 +37,7 @@ struct DecArgs {
   const float *P;                // flat parameters
   DecLayout L;
   size_t W_1, b_1, w_2, b_2;
-  int k, heads, d_h;
+  int k, heads, d_h, B;
   float slope;
   float *r, *c, *yhat;           // [B][k·D], [B][d_h], [B]
 };
@@ -57,8 +57,8 @@ __device__ void warp_gemv(const float *__restrict__ W, int ldw, int ncols, int n
                           const float *X, int ldx, int nvec, float *Y, int ldy,
                           const float *__restrict__ bias, bool relu) {
   constexpr int RB = 8;
-  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  for (int n0 = warp * RB; n0 < nrows; n0 += NW * RB) {
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, nw = blockDim.x >> 5;
+  for (int n0 = warp * RB; n0 < nrows; n0 += nw * RB) {
     for (int c0 = 0; c0 < ncols; c0 += 128) {
       const int c = c0 + lane * 4;
       float4 w[RB];
@@ -94,13 +94,69 @@ __device__ void warp_gemv(const float *__restrict__ W, int ldw, int ncols, int n
   }
 }
 
+// Butterfly GEMV for the decoder tail (ncols <= 128, nvec <= 8): Y[v·ldy + n] = act(bias[n] +
+// Σ_c W[n·ldw + c] X[v·ldx + c]).  A warp takes RB = 32 / NV rows at once (NV = nvec rounded up
+// to a power of two, the padding vectors are zero); lane = 4 columns; the 32 (row, vector)
+// partial dots are reduced across the warp by a butterfly reduce-scatter (31 shuffles instead of
+// 32 x 5), after which lane l holds output l = q·NV + v.  Fixed order (deterministic).
+template <int NV>
+__device__ void warp_gemv_bf(const float *__restrict__ W, int ldw, int ncols, int nrows,
+                             const float *X, int ldx, int nvec, float *Y, int ldy,
+                             const float *__restrict__ bias, bool relu) {
+  constexpr int RB = 32 / NV;
+  const int nw = blockDim.x >> 5, warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int c = lane * 4;
+  float4 x[NV];
+#pragma unroll
+  for (int v = 0; v < NV; ++v)
+    x[v] = (v < nvec && c < ncols) ? *reinterpret_cast<const float4 *>(X + v * ldx + c)
+                                   : make_float4(0.f, 0.f, 0.f, 0.f);
+  for (int n0 = warp * RB; n0 < nrows; n0 += nw * RB) {
+    float val[32];
+#pragma unroll
+    for (int q = 0; q < RB; ++q) {
+      const int n = min(n0 + q, nrows - 1);
+      const float4 w = c < ncols ? __ldg(reinterpret_cast<const float4 *>(W + long(n) * ldw + c))
+                                 : make_float4(0.f, 0.f, 0.f, 0.f);
+#pragma unroll
+      for (int v = 0; v < NV; ++v)
+        val[q * NV + v] = fmaf(w.x, x[v].x, fmaf(w.y, x[v].y, fmaf(w.z, x[v].z, w.w * x[v].w)));
+    }
+#pragma unroll
+    for (int half = 16; half >= 1; half >>= 1) {
+      const bool up = (lane & half) != 0;
+#pragma unroll
+      for (int i = 0; i < half; ++i) {
+        const float send = up ? val[i] : val[i + half];
+        const float keep = up ? val[i + half] : val[i];
+        val[i] = keep + __shfl_xor_sync(0xffffffffu, send, half);
+      }
+    }
+    const int q = lane / NV, v = lane % NV, n = n0 + q;
+    if (v < nvec && n < nrows) {
+      const float a = val[0] + (bias ? __ldg(bias + n) : 0.f);
+      Y[v * ldy + n] = relu ? fmaxf(a, 0.f) : a;
+    }
+  }
+}
+
+// dispatch on the vector count (k seeds per graph, <= 8)
+__device__ __forceinline__ void gemv_k(const float *__restrict__ W, int ldw, int ncols, int nrows,
+                                       const float *X, int ldx, int nvec, float *Y, int ldy,
+                                       const float *__restrict__ bias, bool relu) {
+  if (nvec <= 1) warp_gemv_bf<1>(W, ldw, ncols, nrows, X, ldx, nvec, Y, ldy, bias, relu);
+  else if (nvec <= 2) warp_gemv_bf<2>(W, ldw, ncols, nrows, X, ldx, nvec, Y, ldy, bias, relu);
+  else if (nvec <= 4) warp_gemv_bf<4>(W, ldw, ncols, nrows, X, ldx, nvec, Y, ldy, bias, relu);
+  else warp_gemv_bf<8>(W, ldw, ncols, nrows, X, ldx, nvec, Y, ldy, bias, relu);
+}
+
 // Y[v] = LN(A[v] + Bv[v]) · g + b over D channels (eps 1e-5, biased variance); warp per vector.
 template <int D>
 __device__ void warp_add_ln(const float *A, const float *Bv, float *Y, int nvec,
                             const float *__restrict__ g, const float *__restrict__ b) {
   constexpr int V = D / 32;
-  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  for (int v = warp; v < nvec; v += NW) {
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, nw = blockDim.x >> 5;
+  for (int v = warp; v < nvec; v += nw) {
     float x[V], s = 0.f;
 #pragma unroll
     for (int i = 0; i < V; ++i) {
@@ -158,27 +214,30 @@ __global__ void __launch_bounds__(DT) set_decoder_prep_kernel(const DecArgs a, f
   }
 }
 
+// Pool (PMA's attention of the k seeds over the graph's nodes), split over SPLIT contiguous
+// node ranges per graph: CTA (g, s) writes its unnormalised online-softmax state
+// (running max m, sum l, Σ 2^{(score - m)·log2e} Z) per (seed, head) to part.
+constexpr int SPLIT = 8;
 template <int D>
-__global__ void __launch_bounds__(DT) set_decoder_kernel(const DecArgs a, const float *__restrict__ prep) {
+constexpr int part_stride() { return KHMAX * D + 2 * KHMAX; }
+
+template <int D>
+__global__ void __launch_bounds__(DT) set_decoder_pool_kernel(const DecArgs a, const float *__restrict__ prep,
+                                                              float *__restrict__ part) {
   extern __shared__ __align__(16) float sm[];
-  const int k = a.k, heads = a.heads, KH = k * heads, dh = D / heads;
+  const int k = a.k, heads = a.heads, KH = k * heads;
   float *Zc = sm;                          // [CH][D]
   float *sc = Zc + CH * D;                 // [CH][KHMAX]  scores, then weights
   float *Msm = sc + CH * KHMAX;            // [CH][NW][KHMAX] score partials
   float *Pacc = Msm + CH * NW * KHMAX;     // [KHMAX][D]
-  float *buf = Pacc + KHMAX * D;           // 6 x [KMAX][D]
-  float *B0 = buf, *B1 = B0 + KMAX * D, *B2 = B1 + KMAX * D, *B3 = B2 + KMAX * D,
-        *B4 = B3 + KMAX * D, *B5 = B4 + KMAX * D;
-  float *cst = B5 + KMAX * D;              // [KHMAX]
+  float *cst = Pacc + KHMAX * D;           // [KHMAX]
   float *mrun = cst + KHMAX, *lrun = mrun + KHMAX, *scl = lrun + KHMAX;
-  float *cvec = scl + KHMAX;               // [d_h]
   const int t = threadIdx.x;
-  const float *P = a.P;
-  const DecLayout &L = a.L;
-  const int g = blockIdx.x;
-  const long u0 = a.node_off[g], u1 = a.node_off[g + 1];
+  const int g = blockIdx.x, sp = blockIdx.y;
   pdl_trigger();
   pdl_wait();
+  const long g0 = a.node_off[g], len = a.node_off[g + 1] - g0;
+  const long u0 = g0 + len * sp / SPLIT, u1 = g0 + len * (sp + 1) / SPLIT;
 
   // ---- the folded key map M, c of the seeds' queries (set_decoder_prep_kernel, R32);
   // thread t keeps M[cg·CPG .. +CPG][t & 15] in registers for the score dots
@@ -188,7 +247,6 @@ __global__ void __launch_bounds__(DT) set_decoder_kernel(const DecArgs a, const 
 #pragma unroll
   for (int i = 0; i < CPG; ++i) mreg[i] = __ldg(prep + (cg * CPG + i) * KHMAX + (t & 15));
   float *red = Msm;                        // [CH][NW][KHMAX] score partials (M lives in registers)
-  const float isq = rsqrtf(float(dh));
   if (t < KH) {
     cst[t] = prep[D * KHMAX + t];
     mrun[t] = -INFINITY;
@@ -267,40 +325,103 @@ __global__ void __launch_bounds__(DT) set_decoder_kernel(const DecArgs a, const 
     }
     __syncthreads();
   }
-  for (int o = t; o < KH * D; o += DT) Pacc[o] = Pacc[o] / lrun[o / D];
+  float *out = part + (long(g) * SPLIT + sp) * part_stride<D>();
+  for (int o = t; o < KH * D; o += DT) out[o] = Pacc[o];
+  if (t < KH) {
+    out[KHMAX * D + t] = mrun[t];
+    out[KHMAX * D + KHMAX + t] = lrun[t];
+  }
+}
+
+// GPC graphs per CTA: combine each graph's SPLIT pool partials in fixed order, then the
+// MAB / SAB / FFN chain and the head as GEMVs over all GPC·k vectors of the CTA (every weight
+// row read from L2 once per CTA serves GPC graphs).
+constexpr int GPC = 1;
+constexpr int DT_TAIL = 256;   // tail CTA: 8 warps (all B CTAs resident at once)
+template <int D>
+constexpr size_t tail_smem_floats(int d_h) {
+  return size_t(GPC) * (KMAX * KMAX * 8 + KHMAX * D + 6 * KMAX * D + SPLIT * KHMAX + KHMAX + d_h);
+}
+
+template <int D>
+__global__ void __launch_bounds__(DT_TAIL) set_decoder_kernel(const DecArgs a, const float *__restrict__ part) {
+  extern __shared__ __align__(16) float sm[];
+  const int k = a.k, heads = a.heads, KH = k * heads, dh = D / heads;
+  const int g0 = blockIdx.x * GPC;
+  const int G = min(GPC, a.B - g0);          // graphs of this CTA
+  const int V = G * k;                       // vectors of the CTA ([graph][seed])
+  float *Zc = sm;                            // [GPC][heads][k][k] SAB scores
+  float *Pacc = Zc + GPC * KMAX * KMAX * 8;  // [GPC][KH][D]
+  float *buf = Pacc + GPC * KHMAX * D;       // 6 x [GPC·k][D]
+  constexpr int BS = GPC * KMAX * D;
+  float *B0 = buf, *B1 = B0 + BS, *B2 = B1 + BS, *B3 = B2 + BS, *B4 = B3 + BS, *B5 = B4 + BS;
+  float *fs = B5 + BS;                       // [GPC][SPLIT][KHMAX] partial scale factors
+  float *lsum = fs + GPC * SPLIT * KHMAX;    // [GPC][KHMAX]
+  float *cvec = lsum + GPC * KHMAX;          // [GPC][d_h]
+  const int t = threadIdx.x;
+  const float *P = a.P;
+  const DecLayout &L = a.L;
+  const float isq = rsqrtf(float(dh));
+  pdl_trigger();
+  pdl_wait();
+  constexpr int PS = part_stride<D>();
+  for (int o = t; o < G * KH; o += DT_TAIL) {     // global max, factors 2^{(m_s - M)·log2e}, total sum
+    const int gg = o / KH, kh = o % KH;
+    const float *pg = part + long(g0 + gg) * SPLIT * PS;
+    float M = -INFINITY;
+    for (int q = 0; q < SPLIT; ++q) M = fmaxf(M, pg[q * PS + KHMAX * D + kh]);
+    float l = 0.f;
+    for (int q = 0; q < SPLIT; ++q) {
+      const float mq = pg[q * PS + KHMAX * D + kh];
+      const float f = mq == -INFINITY ? 0.f : ex2((mq - M) * L2E);
+      fs[(gg * SPLIT + q) * KHMAX + kh] = f;
+      l = fmaf(pg[q * PS + KHMAX * D + KHMAX + kh], f, l);
+    }
+    lsum[gg * KHMAX + kh] = l;
+  }
+  __syncthreads();
+  for (int o = t; o < G * KH * D; o += DT_TAIL) {
+    const int gg = o / (KH * D), r = o % (KH * D), kh = r / D;
+    const float *pg = part + long(g0 + gg) * SPLIT * PS;
+    float acc = 0.f;
+    for (int q = 0; q < SPLIT; ++q) acc = fmaf(pg[q * PS + r], fs[(gg * SPLIT + q) * KHMAX + kh], acc);
+    Pacc[o] = acc / lsum[gg * KHMAX + kh];    // [gg][kh][c] = [(gg·k + j)·heads + h][c]
+  }
   __syncthreads();
 
   // ---- MAB1 = PMA_k: O = W_v P + b_v per head, X1 = W_o O + b_o, H̄ = LN(S + X1), LN(H̄ + FFN(H̄))
   for (int h = 0; h < heads; ++h)
-    warp_gemv(P + L.M1.Wv + long(h) * dh * D, D, D, dh, Pacc + h * D, heads * D, k, B0 + h * dh, D,
+    gemv_k(P + L.M1.Wv + long(h) * dh * D, D, D, dh, Pacc + h * D, heads * D, V, B0 + h * dh, D,
               P + L.M1.bv + h * dh, false);
   __syncthreads();
-  warp_gemv(P + L.M1.Wo, D, D, D, B0, D, k, B1, D, P + L.M1.bo, false);
-  for (int i = t; i < k * D; i += DT) B3[i] = P[L.S + i];
+  gemv_k(P + L.M1.Wo, D, D, D, B0, D, V, B1, D, P + L.M1.bo, false);
+  for (int i = t; i < V * D; i += DT_TAIL) B3[i] = P[L.S + i % (k * D)];
   __syncthreads();
-  warp_add_ln<D>(B3, B1, B2, k, P + L.M1.ln1_g, P + L.M1.ln1_b);      // B2 = H̄1
+  warp_add_ln<D>(B3, B1, B2, V, P + L.M1.ln1_g, P + L.M1.ln1_b);      // B2 = H̄1
   __syncthreads();
-  warp_gemv(P + L.M1.F.W1, D, D, D, B2, D, k, B3, D, P + L.M1.F.b1, true);
+  gemv_k(P + L.M1.F.W1, D, D, D, B2, D, V, B3, D, P + L.M1.F.b1, true);
   __syncthreads();
-  warp_gemv(P + L.M1.F.W2, D, D, D, B3, D, k, B4, D, P + L.M1.F.b2, false);
+  gemv_k(P + L.M1.F.W2, D, D, D, B3, D, V, B4, D, P + L.M1.F.b2, false);
   __syncthreads();
-  warp_add_ln<D>(B2, B4, B5, k, P + L.M1.ln2_g, P + L.M1.ln2_b);      // B5 = PMA_k(Z)
+  warp_add_ln<D>(B2, B4, B5, V, P + L.M1.ln2_g, P + L.M1.ln2_b);      // B5 = PMA_k(Z)
   __syncthreads();
 
-  // ---- MAB2 = SAB over the k vectors
-  warp_gemv(P + L.M2.Wq, D, D, D, B5, D, k, B0, D, P + L.M2.bq, false);
-  warp_gemv(P + L.M2.Wk, D, D, D, B5, D, k, B1, D, P + L.M2.bk, false);
-  warp_gemv(P + L.M2.Wv, D, D, D, B5, D, k, B2, D, P + L.M2.bv, false);
+  // ---- MAB2 = SAB over each graph's k vectors
+  gemv_k(P + L.M2.Wq, D, D, D, B5, D, V, B0, D, P + L.M2.bq, false);
+  gemv_k(P + L.M2.Wk, D, D, D, B5, D, V, B1, D, P + L.M2.bk, false);
+  gemv_k(P + L.M2.Wv, D, D, D, B5, D, V, B2, D, P + L.M2.bv, false);
   __syncthreads();
-  // scores / softmax over the k keys per (head, query); Zc reused as [heads][k][k]
-  for (int o = t; o < heads * k * k; o += DT) {
-    const int h = o / (k * k), j = (o / k) % k, jj = o % k;
+  const int HKK = heads * k * k;
+  for (int o = t; o < G * HKK; o += DT_TAIL) {     // scores per (graph, head, query, key)
+    const int gg = o / HKK, r = o % HKK;
+    const int h = r / (k * k), j = (r / k) % k, jj = r % k;
+    const float *qv = B0 + (gg * k + j) * D + h * dh, *kv = B1 + (gg * k + jj) * D + h * dh;
     float s = 0.f;
-    for (int i = 0; i < dh; ++i) s = fmaf(B0[j * D + h * dh + i], B1[jj * D + h * dh + i], s);
+    for (int i = 0; i < dh; ++i) s = fmaf(qv[i], kv[i], s);
     Zc[o] = s * isq;
   }
   __syncthreads();
-  for (int o = t; o < heads * k; o += DT) {
+  for (int o = t; o < G * heads * k; o += DT_TAIL) {   // softmax over the k keys
     float m = -INFINITY, l = 0.f;
     for (int jj = 0; jj < k; ++jj) m = fmaxf(m, Zc[o * k + jj]);
     for (int jj = 0; jj < k; ++jj) {
@@ -311,42 +432,45 @@ __global__ void __launch_bounds__(DT) set_decoder_kernel(const DecArgs a, const 
     for (int jj = 0; jj < k; ++jj) Zc[o * k + jj] /= l;
   }
   __syncthreads();
-  for (int o = t; o < k * D; o += DT) {
-    const int j = o / D, ch = o % D, h = ch / dh;
+  for (int o = t; o < V * D; o += DT_TAIL) {
+    const int v = o / D, gg = v / k, j = v % k, ch = o % D, h = ch / dh;
+    const float *w = Zc + gg * HKK + (h * k + j) * k;
     float acc = 0.f;
-    for (int jj = 0; jj < k; ++jj) acc = fmaf(Zc[(h * k + j) * k + jj], B2[jj * D + ch], acc);
+    for (int jj = 0; jj < k; ++jj) acc = fmaf(w[jj], B2[(gg * k + jj) * D + ch], acc);
     B3[o] = acc;
   }
   __syncthreads();
-  warp_gemv(P + L.M2.Wo, D, D, D, B3, D, k, B4, D, P + L.M2.bo, false);
+  gemv_k(P + L.M2.Wo, D, D, D, B3, D, V, B4, D, P + L.M2.bo, false);
   __syncthreads();
-  warp_add_ln<D>(B5, B4, B0, k, P + L.M2.ln1_g, P + L.M2.ln1_b);      // B0 = H̄2
+  warp_add_ln<D>(B5, B4, B0, V, P + L.M2.ln1_g, P + L.M2.ln1_b);      // B0 = H̄2
   __syncthreads();
-  warp_gemv(P + L.M2.F.W1, D, D, D, B0, D, k, B1, D, P + L.M2.F.b1, true);
+  gemv_k(P + L.M2.F.W1, D, D, D, B0, D, V, B1, D, P + L.M2.F.b1, true);
   __syncthreads();
-  warp_gemv(P + L.M2.F.W2, D, D, D, B1, D, k, B2, D, P + L.M2.F.b2, false);
+  gemv_k(P + L.M2.F.W2, D, D, D, B1, D, V, B2, D, P + L.M2.F.b2, false);
   __syncthreads();
-  warp_add_ln<D>(B0, B2, B3, k, P + L.M2.ln2_g, P + L.M2.ln2_b);      // B3 = SAB(PMA_k(Z))
+  warp_add_ln<D>(B0, B2, B3, V, P + L.M2.ln2_g, P + L.M2.ln2_b);      // B3 = SAB(PMA_k(Z))
   __syncthreads();
 
-  // ---- final FFN -> decoder output [k][D] (flattened into r), then the head
-  warp_gemv(P + L.D.W1, D, D, D, B3, D, k, B4, D, P + L.D.b1, true);
+  // ---- final FFN -> decoder output [k][D] per graph (flattened into r), then the head
+  gemv_k(P + L.D.W1, D, D, D, B3, D, V, B4, D, P + L.D.b1, true);
   __syncthreads();
-  warp_gemv(P + L.D.W2, D, D, D, B4, D, k, B5, D, P + L.D.b2, false);
+  gemv_k(P + L.D.W2, D, D, D, B4, D, V, B5, D, P + L.D.b2, false);
   __syncthreads();
-  for (int i = t; i < k * D; i += DT) a.r[long(g) * k * D + i] = B5[i];
-  warp_gemv(P + a.W_1, k * D, k * D, a.d_h, B5, 0, 1, cvec, 0, P + a.b_1, false);
+  for (int i = t; i < V * D; i += DT_TAIL) a.r[long(g0) * k * D + i] = B5[i];
+  warp_gemv(P + a.W_1, k * D, k * D, a.d_h, B5, k * D, G, cvec, a.d_h, P + a.b_1, false);
   __syncthreads();
-  if (t < 32) {        // ŷ = w_2 · LReLU(c) + b_2, fixed-order warp reduction
+  const int warp = t >> 5, lane = t & 31;
+  if (warp < G) {      // ŷ = w_2 · LReLU(c) + b_2, fixed-order warp reduction, warp per graph
+    const int g = g0 + warp;
     float s = 0.f;
-    for (int i = t; i < a.d_h; i += 32) {
-      const float cv = cvec[i];
+    for (int i = lane; i < a.d_h; i += 32) {
+      const float cv = cvec[warp * a.d_h + i];
       a.c[long(g) * a.d_h + i] = cv;
       s = fmaf(__ldg(P + a.w_2 + i), cv > 0.f ? cv : a.slope * cv, s);
     }
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
-    if (t == 0) a.yhat[g] = s + __ldg(P + a.b_2);
+    if (lane == 0) a.yhat[g] = s + __ldg(P + a.b_2);
   }
 }
 
@@ -364,29 +488,45 @@ int launch_set_decoder(const occu_ctx *ctx, const DevCsr &csr, const float *hL, 
   if ((rr = launch_bias_tc(ctx, T, cf.d, csr.N, 1, cf.L, P + L.D.P.b2, false, Z, "dec_ffn_tc", st)) < 0) return rr;
   n += rr;
   DecArgs a{};
+  if (!ctx->ws.dprep.ptr) const_cast<occu_ctx *>(ctx)->dprep_version = -1;   // fresh buffer
   if (const_cast<occu_ctx *>(ctx)->ws.dprep.ensure(size_t(cf.d * KHMAX + KHMAX) * 4) != cudaSuccess)
     return -int(cudaErrorMemoryAllocation);
   float *prep = ctx->ws.dprep.as<float>();
   a.Z = Z; a.node_off = csr.node_off; a.P = P; a.L = L.D;
   a.W_1 = L.W_1; a.b_1 = L.b_1; a.w_2 = L.w_2; a.b_2 = L.b_2;
-  a.k = cf.k; a.heads = cf.heads; a.d_h = cf.d_h; a.slope = cf.slope;
+  a.k = cf.k; a.heads = cf.heads; a.d_h = cf.d_h; a.slope = cf.slope; a.B = csr.B;
   a.r = r; a.c = c; a.yhat = yhat;
   const int D = cf.d;
-  const size_t smem = size_t(CH * D + CH * KHMAX + CH * NW * KHMAX + KHMAX * D + 6 * KMAX * D +
-                             4 * KHMAX + cf.d_h) * 4;
-  OCCU_PROF_BEGIN(ctx, "set_decoder", st);
-  if (D == 64) {
-    set_decoder_prep_kernel<64><<<1, DT, 0, st>>>(a, prep);
-    cudaFuncSetAttribute(set_decoder_kernel<64>, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
-    launch_pdl(ctx->pdl & 8, set_decoder_kernel<64>, csr.B, DT, smem, st, a, (const float *)prep);
-  } else {
-    set_decoder_prep_kernel<128><<<1, DT, 0, st>>>(a, prep);
-    cudaFuncSetAttribute(set_decoder_kernel<128>, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
-    launch_pdl(ctx->pdl & 8, set_decoder_kernel<128>, csr.B, DT, smem, st, a, (const float *)prep);
-  }
-  OCCU_PROF_END(ctx);
+  if (const_cast<occu_ctx *>(ctx)->ws.dpool.ensure(size_t(csr.B) * SPLIT * (KHMAX * D + 2 * KHMAX) * 4) != cudaSuccess)
+    return -int(cudaErrorMemoryAllocation);
+  float *part = ctx->ws.dpool.as<float>();
+  const size_t smem_pool = size_t(CH * D + CH * KHMAX + CH * NW * KHMAX + KHMAX * D + 4 * KHMAX) * 4;
+  const size_t smem_tail = (D == 64 ? tail_smem_floats<64>(cf.d_h) : tail_smem_floats<128>(cf.d_h)) * 4;
+  const dim3 gpool(csr.B, SPLIT);
+  int nprep = 0;
+  auto run = [&](auto prepk, auto poolk, auto tailk) {
+    if (ctx->dprep_version != ctx->params_version) {   // parameters changed: rebuild M, c
+      OCCU_PROF_BEGIN(ctx, "set_decoder_prep", st);
+      prepk<<<1, DT, 0, st>>>(a, prep);
+      OCCU_PROF_END(ctx);
+      const_cast<occu_ctx *>(ctx)->dprep_version = ctx->params_version;
+      ++nprep;
+    }
+    OCCU_PROF_BEGIN(ctx, "set_decoder_pool", st);
+    cudaFuncSetAttribute(poolk, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem_pool));
+    launch_pdl(ctx->pdl & 8, poolk, gpool, DT, smem_pool, st, a, (const float *)prep, part);
+    OCCU_PROF_END(ctx);
+    OCCU_PROF_BEGIN(ctx, "set_decoder", st);
+    cudaFuncSetAttribute(tailk, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem_tail));
+    launch_pdl(ctx->pdl & 8, tailk, (csr.B + GPC - 1) / GPC, DT_TAIL, smem_tail, st, a, (const float *)part);
+    OCCU_PROF_END(ctx);
+  };
+  if (D == 64)
+    run(set_decoder_prep_kernel<64>, set_decoder_pool_kernel<64>, set_decoder_kernel<64>);
+  else
+    run(set_decoder_prep_kernel<128>, set_decoder_pool_kernel<128>, set_decoder_kernel<128>);
   const cudaError_t e = cudaGetLastError();
-  return e == cudaSuccess ? n + 2 : -int(e);
+  return e == cudaSuccess ? n + 2 + nprep : -int(e);
 }
 
 }  // namespace occu

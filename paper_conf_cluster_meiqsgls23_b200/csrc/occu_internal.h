@@ -66,6 +66,7 @@ struct Workspace {
   DevBuf anf[2], aef[2], acsr[2];   // occu_predict_async: double-buffered input staging
   DevBuf dT, dZ;           // decoder readout: per-node FFN hidden / output rows [N][d]
   DevBuf dprep;            // decoder readout: folded key map M [d][16] and offsets c [16]
+  DevBuf dpool;            // decoder readout: pool partials [B][8][16·d + 32]
   std::vector<DevBuf> gh;  // Graphormer layer outputs [N][d] (per layer)
   DevBuf gx, gqkv, go;     // Graphormer scratch: LN output [N][d], Q|K|V [3][N][d], attention [N][d]
   void release_all();
@@ -116,6 +117,7 @@ struct occu_ctx {
   int fuse_edge_gate = 0;  // path 0: edge transform + gate in one kernel (edgegate_kernel), OCCU_FUSE_EG=1
   occu::DevBuf wimg, wjobs, wfexp;   // prebuilt tensor-core weight images (per parameter version)
   int64_t params_version = 0, wimg_version = -1;
+  int64_t dprep_version = -1;   // decoder: params version the folded key map was built for
   float weight_decay = 1e-4f;
   occu::DevBuf params, grads, adam_m, adam_v;
   int64_t adam_t = 0;
