@@ -26,6 +26,7 @@
 #include <stdint.h>
 
 #include "occu_internal.h"
+#include "tc_common.cuh"
 
 namespace occu {
 namespace {
@@ -557,6 +558,217 @@ __global__ void __launch_bounds__(AW * 32) gph_attn_f16_kernel(const AttnArgs a)
   }
 }
 
+// ---- tcgen05 variant (d_h = 32): CTA = 128 query rows x one head, thread = query row = TMEM
+// lane.  Q (scaled, fp16x2 split) lives in TMEM as the A operand; per 64-key block the CTA
+// splits K into fp16 hi / lo SW128 tiles (B of S = Q·Kᵀ, N = 64) and V transposed into SW128
+// tiles (B of O += P·V, N = 32, K = 64 keys); one thread issues 3 tcgen05.mma per K step for
+// each product (hi·hi + hi·lo + lo·hi, FP32 accumulation in TMEM).  Each thread reads its
+// row of S from TMEM (masking keys outside its graph), runs the online softmax, writes P hi / lo
+// back to TMEM as the A operand of P·V and rescales its O row in TMEM.  Steps are serialised
+// inside a CTA; two CTAs per SM (256 TMEM columns each) overlap one another.
+namespace gtc {
+constexpr int KB = 64;                       // keys per block
+constexpr uint32_t TCOLS = 128;
+// TMEM columns: Q hi / lo (16 each), S (64; P hi / lo overwrite it once the row is read), O (32)
+constexpr uint32_t QH = 0, QL = 16, SC = 32, PH = 32, PL = 64, OC = 96;
+constexpr uint32_t K_BYTES = KB * 128, V_BYTES = 32 * 128;
+constexpr size_t SMEM = 50 * 1024;           // caps residency at four CTAs per SM (TMEM budget)
+}
+
+// spin (no back-off sleep): the waits here are short MMAs on the critical path
+__device__ __forceinline__ void mbar_spin(uint64_t *bar, uint32_t parity) {
+  const uint32_t a = tc::smem_u32(bar);
+  while (!tc::mbar_try_wait(a, parity)) {
+  }
+}
+
+__device__ __forceinline__ void fence_proxy_async_smem() {
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+}
+
+__global__ void __launch_bounds__(128) gph_attn_tc_kernel(const AttnArgs a) {
+  using namespace gtc;
+  extern __shared__ __align__(1024) uint8_t gsm_raw[];
+  uint8_t *sm = gsm_raw + ((1024u - (tc::smem_u32(gsm_raw) & 1023u)) & 1023u);
+  uint8_t *Kh = sm, *Kl = sm + K_BYTES, *Vh = sm + 2 * K_BYTES, *Vl = Vh + V_BYTES;
+  uint64_t *bar = reinterpret_cast<uint64_t *>(Vl + V_BYTES);
+  uint32_t *slot = reinterpret_cast<uint32_t *>(bar + 1);
+  const int t = threadIdx.x, warp = t >> 5, lane = t & 31;
+  const long q0 = long(blockIdx.x) * 128;
+  const int D = a.D;
+  const long hc = long(blockIdx.y) * 32;
+  pdl_trigger();
+  if (warp == 0) tc::tmem_alloc<TCOLS>(slot);
+  if (t == 0) {
+    tc::mbar_init(bar, 1);
+    tc::fence_mbar_init();
+  }
+  tc::fence_before_sync();
+  __syncthreads();
+  tc::fence_after_sync();
+  const uint32_t tmem = *slot;
+  const uint32_t lane_base = tmem + (uint32_t(warp * 32) << 16);
+
+  const long r = q0 + t;
+  const bool live = r < a.N;
+  const long qlast = min(q0 + 128, long(a.N)) - 1;
+  const int kbeg = __ldg(a.node_off + __ldg(a.node_graph + q0));
+  const int kend = __ldg(a.node_off + __ldg(a.node_graph + qlast) + 1);
+  int lo = 0, hi = 0;
+  if (live) {
+    const int gr = __ldg(a.node_graph + r);
+    lo = __ldg(a.node_off + gr);
+    hi = __ldg(a.node_off + gr + 1);
+  }
+  {   // Q row -> TMEM (scaled, fp16x2 split); O row = 0
+    uint32_t qh[16], ql[16], z[32];
+#pragma unroll
+    for (int c = 0; c < 32; c += 4) {
+      float4 x = make_float4(0.f, 0.f, 0.f, 0.f);
+      if (live) x = __ldg(reinterpret_cast<const float4 *>(a.Q + r * D + hc + c));
+      split_h2(x.x * a.qscale, x.y * a.qscale, qh[c / 2], ql[c / 2]);
+      split_h2(x.z * a.qscale, x.w * a.qscale, qh[c / 2 + 1], ql[c / 2 + 1]);
+    }
+#pragma unroll
+    for (int c = 0; c < 32; ++c) z[c] = 0u;
+    tc::tmem_st16(lane_base + QH, qh);
+    tc::tmem_st16(lane_base + QL, ql);
+    tc::tmem_st32(lane_base + OC, z);
+    tc::tmem_st_wait();
+  }
+  const uint32_t kh_a = tc::smem_u32(Kh), kl_a = tc::smem_u32(Kl), vh_a = tc::smem_u32(Vh),
+                 vl_a = tc::smem_u32(Vl);
+  const uint32_t id_s = tc::idesc(128, KB, tc::FMT_F16), id_o = tc::idesc(128, 32, tc::FMT_F16);
+  float m = -INFINITY, l = 0.f;
+  uint32_t phase = 0;
+  // staging roles: K row kr = t >> 1, dims d0 .. d0 + 15; Vᵀ row = dim `lane`, keys w·16 .. + 15
+  const int kr = t >> 1, d0 = (t & 1) * 16, vk0 = warp * 16;
+  float4 kx[4];
+  float vx[16];
+  auto load_block = [&](int kb) {
+    const long key = long(kb) + kr;
+    const bool ok = key < kend;
+#pragma unroll
+    for (int c = 0; c < 4; ++c)
+      kx[c] = ok ? __ldg(reinterpret_cast<const float4 *>(a.K + key * D + hc + d0) + c)
+                 : make_float4(0.f, 0.f, 0.f, 0.f);
+#pragma unroll
+    for (int c = 0; c < 16; ++c) {
+      const long kv = long(kb) + vk0 + c;
+      vx[c] = kv < kend ? __ldg(a.V + kv * D + hc + lane) : 0.f;
+    }
+  };
+  if (kbeg < kend) load_block(kbeg);
+  for (int kb = kbeg; kb < kend; kb += KB) {
+    {   // ---- stage the prefetched block: K (SW128 K-major, rows = keys), Vᵀ (rows = dims)
+      uint32_t h[8], lw[8];
+#pragma unroll
+      for (int c = 0; c < 4; ++c) {
+        split_h2(kx[c].x, kx[c].y, h[2 * c], lw[2 * c]);
+        split_h2(kx[c].z, kx[c].w, h[2 * c + 1], lw[2 * c + 1]);
+      }
+      *reinterpret_cast<uint4 *>(Kh + tc::sw128_offset_f16(kr, d0, KB)) = make_uint4(h[0], h[1], h[2], h[3]);
+      *reinterpret_cast<uint4 *>(Kh + tc::sw128_offset_f16(kr, d0 + 8, KB)) = make_uint4(h[4], h[5], h[6], h[7]);
+      *reinterpret_cast<uint4 *>(Kl + tc::sw128_offset_f16(kr, d0, KB)) = make_uint4(lw[0], lw[1], lw[2], lw[3]);
+      *reinterpret_cast<uint4 *>(Kl + tc::sw128_offset_f16(kr, d0 + 8, KB)) = make_uint4(lw[4], lw[5], lw[6], lw[7]);
+#pragma unroll
+      for (int c = 0; c < 8; ++c) split_h2(vx[2 * c], vx[2 * c + 1], h[c], lw[c]);
+      *reinterpret_cast<uint4 *>(Vh + tc::sw128_offset_f16(lane, vk0, 32)) = make_uint4(h[0], h[1], h[2], h[3]);
+      *reinterpret_cast<uint4 *>(Vh + tc::sw128_offset_f16(lane, vk0 + 8, 32)) = make_uint4(h[4], h[5], h[6], h[7]);
+      *reinterpret_cast<uint4 *>(Vl + tc::sw128_offset_f16(lane, vk0, 32)) = make_uint4(lw[0], lw[1], lw[2], lw[3]);
+      *reinterpret_cast<uint4 *>(Vl + tc::sw128_offset_f16(lane, vk0 + 8, 32)) = make_uint4(lw[4], lw[5], lw[6], lw[7]);
+    }
+    fence_proxy_async_smem();
+    tc::fence_before_sync();
+    __syncthreads();
+    tc::fence_after_sync();
+    if (t == 0) {     // ---- S = Q Kᵀ (N = 64, K = 32: two k16 steps)
+#pragma unroll
+      for (int kk = 0; kk < 2; ++kk) {
+        const uint64_t bh = tc::sdesc_sw128(kh_a + kk * 32), bl = tc::sdesc_sw128(kl_a + kk * 32);
+        tc::mma_f16_ts(tmem + SC, tmem + QL + kk * 8, bh, id_s, kk > 0 ? 1u : 0u);
+        tc::mma_f16_ts(tmem + SC, tmem + QH + kk * 8, bl, id_s, 1u);
+        tc::mma_f16_ts(tmem + SC, tmem + QH + kk * 8, bh, id_s, 1u);
+      }
+      tc::mma_commit(bar);
+    }
+    if (kb + KB < kend) load_block(kb + KB);        // next block's K / V in flight meanwhile
+    mbar_spin(bar, phase);
+    phase ^= 1;
+    tc::fence_after_sync();
+    {   // ---- online softmax on this thread's row (P overwrites S in TMEM)
+      uint32_t s0[32], s1[32];
+      tc::tmem_ld32(lane_base + SC, s0);
+      tc::tmem_ld32(lane_base + SC + 32, s1);
+      tc::tmem_ld_wait();
+      float sv[64];
+      float bm = -INFINITY;
+#pragma unroll
+      for (int j = 0; j < 64; ++j) {
+        const float x = __uint_as_float(j < 32 ? s0[j] : s1[j - 32]);
+        const int key = kb + j;
+        sv[j] = (key >= lo && key < hi) ? x : -INFINITY;
+        bm = fmaxf(bm, sv[j]);
+      }
+      const float mn = fmaxf(m, bm);
+      const float ref = mn == -INFINITY ? 0.f : mn;
+      const float f = ex2f(m - ref);
+      m = mn;
+      float sum = 0.f;
+#pragma unroll
+      for (int j = 0; j < 32; ++j) {
+        const float p0 = ex2f(sv[2 * j] - ref), p1 = ex2f(sv[2 * j + 1] - ref);
+        sum += p0 + p1;
+        split_h2(p0, p1, s0[j], s1[j]);
+      }
+      l = l * f + sum;
+      tc::tmem_st32(lane_base + PH, s0);
+      tc::tmem_st32(lane_base + PL, s1);
+      if (__any_sync(0xffffffffu, f != 1.f)) {     // rescale the O row (warp-collective)
+        uint32_t o[32];
+        tc::tmem_ld32(lane_base + OC, o);
+        tc::tmem_ld_wait();
+#pragma unroll
+        for (int c = 0; c < 32; ++c) o[c] = __float_as_uint(__uint_as_float(o[c]) * f);
+        tc::tmem_st32(lane_base + OC, o);
+      }
+      tc::tmem_st_wait();
+    }
+    tc::fence_before_sync();
+    __syncthreads();
+    tc::fence_after_sync();
+    if (t == 0) {     // ---- O += P V (N = 32, K = 64 keys: four k16 steps)
+#pragma unroll
+      for (int kk = 0; kk < 4; ++kk) {
+        const uint64_t bh = tc::sdesc_sw128(vh_a + kk * 32), bl = tc::sdesc_sw128(vl_a + kk * 32);
+        tc::mma_f16_ts(tmem + OC, tmem + PL + kk * 8, bh, id_o, 1u);
+        tc::mma_f16_ts(tmem + OC, tmem + PH + kk * 8, bl, id_o, 1u);
+        tc::mma_f16_ts(tmem + OC, tmem + PH + kk * 8, bh, id_o, 1u);
+      }
+      tc::mma_commit(bar);
+    }
+    mbar_spin(bar, phase);
+    phase ^= 1;
+    tc::fence_after_sync();
+  }
+  {   // ---- O / l -> global
+    uint32_t o[32];
+    tc::tmem_ld32(lane_base + OC, o);
+    tc::tmem_ld_wait();
+    const float il = l > 0.f ? 1.f / l : 0.f;
+    if (live) {
+#pragma unroll
+      for (int c = 0; c < 32; c += 4)
+        *reinterpret_cast<float4 *>(a.O + r * D + hc + c) =
+            make_float4(__uint_as_float(o[c]) * il, __uint_as_float(o[c + 1]) * il,
+                        __uint_as_float(o[c + 2]) * il, __uint_as_float(o[c + 3]) * il);
+    }
+  }
+  tc::fence_before_sync();
+  __syncthreads();
+  if (warp == 0) tc::tmem_dealloc<TCOLS>(tmem);
+}
+
 template <int D>
 int ln_launch(const occu_ctx *ctx, const float *X, int N, const float *g, const float *b, float *Y,
               cudaStream_t st) {
@@ -610,7 +822,15 @@ int launch_graphormer_layer(const occu_ctx *ctx, const DevCsr &csr, int j, const
     cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
     kern<<<grid, AW * 32, smem, st>>>(a);
   };
-  if (tf32) {              // A/B: the TF32-split variant
+  static const bool use_tc = [] {
+    const char *e = getenv("OCCU_GPH_TC");
+    return !e || atoi(e) != 0;
+  }();
+  if (use_tc && dh == 32 && !tf32) {    // tcgen05 path (d_h = 32)
+    cudaFuncSetAttribute(gph_attn_tc_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, int(gtc::SMEM));
+    const dim3 g2((N + 127) / 128, cf.heads);
+    gph_attn_tc_kernel<<<g2, 128, gtc::SMEM, st>>>(a);
+  } else if (tf32) {       // A/B: the TF32-split variant
     switch (dh) {
       case 16: go(gph_attn_kernel<16>, 16); break;
       case 32: go(gph_attn_kernel<32>, 32); break;
