@@ -703,12 +703,20 @@ __global__ void __launch_bounds__(128) gph_attn_tc_kernel(const AttnArgs a) {
       tc::tmem_ld_wait();
       float sv[64];
       float bm = -INFINITY;
+      if (__all_sync(0xffffffffu, kb >= lo && kb + KB <= hi)) {    // block inside every row's graph
 #pragma unroll
-      for (int j = 0; j < 64; ++j) {
-        const float x = __uint_as_float(j < 32 ? s0[j] : s1[j - 32]);
-        const int key = kb + j;
-        sv[j] = (key >= lo && key < hi) ? x : -INFINITY;
-        bm = fmaxf(bm, sv[j]);
+        for (int j = 0; j < 64; ++j) {
+          sv[j] = __uint_as_float(j < 32 ? s0[j] : s1[j - 32]);
+          bm = fmaxf(bm, sv[j]);
+        }
+      } else {
+#pragma unroll
+        for (int j = 0; j < 64; ++j) {
+          const float x = __uint_as_float(j < 32 ? s0[j] : s1[j - 32]);
+          const int key = kb + j;
+          sv[j] = (key >= lo && key < hi) ? x : -INFINITY;
+          bm = fmaxf(bm, sv[j]);
+        }
       }
       const float mn = fmaxf(m, bm);
       const float ref = mn == -INFINITY ? 0.f : mn;
