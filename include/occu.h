@@ -177,6 +177,39 @@ occu_status occu_compute_grads(occu_ctx *ctx, const occu_batch *batch, const flo
 occu_status occu_get_grads(const occu_ctx *ctx, float *host_flat, size_t n);
 occu_status occu_set_weight_decay(occu_ctx *ctx, float wd);
 
+/* ---- NEXT-4: on-device feature synthesis (R39) ---------
+ * A DL-model family's training DAG has one topology for all its hyperparameter variants
+ * (P237), so a batch of variants is built on the GPU from per-family templates plus four
+ * numbers per graph, instead of copying ~350 B of Table I features per node over PCIe.
+ * occu_template_create uploads one family (device memory of ctx's device, owned by the
+ * template): graph = the family's DAG (host, local ids; validated like occu_pack);
+ * node_static [n][80] = the hyperparameter-independent Table I columns (operator one-hot, role
+ * bits, runtime GPU constants; zeros in columns 42-75); node_coef [n][22][12] = the 22
+ * hyperparameter-dependent quantities of each node (16 operator hyperparameters -> columns
+ * 42-57, 4 tensor sizes -> 66-69 and, times 4 bytes, 70-73, FLOPs -> 74, temporary size -> 75)
+ * as tensor-product Newton coefficients on the nodes batch {4, 8}, cin {1, 2}, seq {16, 32, 48}
+ * (coefficient 6i + 3j + k of Nb_i Nc_j Ns_k, Nb = (1, b-4), Nc = (1, c-1),
+ * Ns = (1, s-16, (s-16)(s-32)); occu_gen/templates.py builds them); edge_static [m][4] (column
+ * 2 zero) and edge_coef [m][12] (bytes carried -> column 2), both in input edge order.
+ * occu_synthesize builds a device batch of num_graphs graphs, graph b = templates[b] at
+ * hp[b] = (batch, cin, seq, hw) (host [B][4], finite, >= 0): the CSR (bit-identical to
+ * occu_pack of the same graphs), node_feat [N][80] and edge_feat [E][4] (input edge order),
+ * each quantity evaluated in float64 and encoded log2(1 + x) / 40 (configuration columns
+ * 58-61 = the encoded hp, 62-65 = 0).  Stream-ordered on the ctx stream.  The returned arrays
+ * live in ctx-owned device memory, valid until the next occu_synthesize on ctx; free the
+ * returned batch struct with occu_batch_free (it does not free the arrays).  Errors:
+ * OCCU_EINVAL (NULL, num_graphs < 1, a template of another device, bad hp, F_n != 80 or
+ * F_e != 4 in the ctx config, N or E >= 2^31), OCCU_ENOMEM, OCCU_ECUDA. */
+typedef struct occu_template occu_template;
+occu_status occu_template_create(occu_ctx *ctx, const occu_graph_view *graph,
+                                 const float *node_static, const double *node_coef,
+                                 const float *edge_static, const double *edge_coef,
+                                 occu_template **out);
+void occu_template_destroy(occu_template *t);
+occu_status occu_synthesize(occu_ctx *ctx, const occu_template *const *templates,
+                            int32_t num_graphs, const float *hp, occu_csr_batch **csr_out,
+                            float **node_feat, float **edge_feat);
+
 /* ---- NEXT-4 consumer: occu-packing (P390-P392; R38) ------------------
  * Host-side first-fit bin packing of jobs by predicted occupancy (the output of
  * occu_predict), the paper's co-location policy: "the cumulative GPU occupancy of the DL

@@ -121,14 +121,19 @@ def mixture_variant(family: str, r: Rng) -> dict:
 MIXTURE = [f for f in dags.FAMILIES if f != "bert_base"]   # the 20 Table II models
 
 
-def mixture(num_graphs: int, seed: int, start: int = 0):
-    """Graphs ``start .. start+num_graphs-1`` of the 20-family mixture (CFG4/CFG5)."""
+def mixture_specs(num_graphs: int, seed: int, start: int = 0):
+    """(family, hp) of graphs ``start .. start+num_graphs-1`` of the 20-family mixture."""
     out = []
     for k in range(start, start + num_graphs):
         r = Rng((seed << 32) + k)
         fam = MIXTURE[int(r.randint(0, len(MIXTURE) - 1)[0])]
         out.append((fam, mixture_variant(fam, r)))
-    return _make(out, seed=seed)
+    return out
+
+
+def mixture(num_graphs: int, seed: int, start: int = 0):
+    """Graphs ``start .. start+num_graphs-1`` of the 20-family mixture (CFG4/CFG5)."""
+    return _make(mixture_specs(num_graphs, seed, start), seed=seed)
 
 
 def random_dag_batch(num_graphs: int, seed: int, max_nodes: int = 12, hub: bool = False,

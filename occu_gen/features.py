@@ -35,11 +35,12 @@ def _enc(x):
     return (np.log2(1.0 + np.asarray(x, dtype=np.float64)) / 40.0)
 
 
-def node_edge_features(g: TrainGraph, hp: dict, gpu: str = "A100"):
-    """Return (node_feat [n,80] f32, edge_feat [m,4] f32) for graph g at hp.
-
-    g.fwd must be the forward builder for the same hp (shapes depend on hp).
-    """
+def node_edge_quantities(g: TrainGraph, hp: dict, gpu: str = "A100"):
+    """The raw (unencoded) per-node / per-edge quantities of Table I for graph g at hp:
+    dict(X = node rows with the hp-independent columns and the configuration columns already
+    encoded, hpn [n,16] operator hyperparameters, sizes [n,4] tensor sizes, f [n] FLOPs,
+    t [n] temporary size, E = edge rows with the constant columns, nbytes [m]).
+    g.fwd must be the forward builder for the same hp (shapes depend on hp)."""
     ops = g.fwd.ops
     nf = len(ops)
     n = g.num_nodes
@@ -100,12 +101,6 @@ def node_edge_features(g: TrainGraph, hp: dict, gpu: str = "A100"):
     sizes[ls, 0] = out_numel[nf - 1]
     sizes[ls, 3] = 1.0
     f[ls] = 3.0 * out_numel[nf - 1]
-    X[:, 42:58] = _enc(hpn)
-    X[:, 66:70] = _enc(sizes)
-    X[:, 70:74] = _enc(4.0 * sizes)
-    X[:, 74] = _enc(f)
-    X[:, 75] = _enc(t)
-
     m = g.num_edges
     E = np.zeros((m, F_E), np.float64)
     E[:, 0] = 1.0 - g.edge_bwd
@@ -114,6 +109,25 @@ def node_edge_features(g: TrainGraph, hp: dict, gpu: str = "A100"):
     upd_edge = g.node_role[g.dst] == ROLE_UPDATE
     if upd_edge.any():
         nbytes[upd_edge] = 4.0 * param_numel[g.node_param[g.dst[upd_edge]]]
-    E[:, 2] = _enc(nbytes)
     E[:, 3] = np.log2(1.0 + bw) / 16.0
+    return dict(X=X, hpn=hpn, sizes=sizes, f=f, t=t, E=E, nbytes=nbytes)
+
+
+def encode_features(q):
+    """Table I encoding of node_edge_quantities' output -> (node_feat f32, edge_feat f32)."""
+    X, E = q["X"].copy(), q["E"].copy()
+    X[:, 42:58] = _enc(q["hpn"])
+    X[:, 66:70] = _enc(q["sizes"])
+    X[:, 70:74] = _enc(4.0 * q["sizes"])
+    X[:, 74] = _enc(q["f"])
+    X[:, 75] = _enc(q["t"])
+    E[:, 2] = _enc(q["nbytes"])
     return X.astype(np.float32), E.astype(np.float32)
+
+
+def node_edge_features(g: TrainGraph, hp: dict, gpu: str = "A100"):
+    """Return (node_feat [n,80] f32, edge_feat [m,4] f32) for graph g at hp.
+
+    g.fwd must be the forward builder for the same hp (shapes depend on hp).
+    """
+    return encode_features(node_edge_quantities(g, hp, gpu))

@@ -68,6 +68,7 @@ struct Workspace {
   DevBuf dprep;            // decoder readout: folded key map M [d][16] and offsets c [16]
   DevBuf dpool;            // decoder readout: pool partials [B][8][16·d + 32]
   std::vector<DevBuf> gh;  // Graphormer layer outputs [N][d] (per layer)
+  DevBuf scsr, snf, sef, sdesc;   // occu_synthesize: batch CSR, node / edge rows, descriptors
   DevBuf gx, gqkv, go;     // Graphormer scratch: LN output [N][d], Q|K|V [3][N][d], attention [N][d]
   void release_all();
 };

@@ -47,7 +47,8 @@ void Workspace::release_all() {
   DevBuf *bufs[] = {&node_feat, &edge_feat, &targets, &out_occ, &csr, &e0, &g, &r, &c, &yhat,
                     &dy, &dc, &dr, &dh, &dhprev, &dP, &MG, &DV, &DZ, &deA, &deB, &dalpha,
                     &dpq, &partial, &loss, &tcpart, &dpart, &rpart, &anf[0], &anf[1],
-                    &aef[0], &aef[1], &acsr[0], &acsr[1], &dT, &dZ, &dprep, &dpool, &gx, &gqkv, &go};
+                    &aef[0], &aef[1], &acsr[0], &acsr[1], &dT, &dZ, &dprep, &dpool, &gx, &gqkv, &go,
+                    &scsr, &snf, &sef, &sdesc};
   for (DevBuf *b : bufs) b->release();
   for (auto *v : {&hbar, &p, &q, &e, &h, &gs, &gh})
     for (DevBuf &b : *v) b.release();

@@ -32,6 +32,7 @@ EXPORTS = [
     "occu_dist_init", "occu_save_state", "occu_load_state", "occu_set_keep_intermediates",
     "occu_get_tensor", "occu_last_launch_count", "occu_last_error", "occu_set_profiling",
     "occu_profile_reset", "occu_profile_query", "occu_set_kernel_path", "occu_pack_jobs",
+    "occu_template_create", "occu_template_destroy", "occu_synthesize",
 ]
 
 
@@ -91,6 +92,9 @@ def lib():
             "occu_get_params": ([VP, VP, SZ], I32),
             "occu_pack": ([P(GraphView), I32, P(P(CsrBatch))], I32),
             "occu_pack_jobs": ([P(C.c_float), I32, C.c_double, P(I32), P(C.c_double), P(I32)], I32),
+            "occu_template_create": ([VP, P(GraphView), VP, VP, VP, VP, P(VP)], I32),
+            "occu_template_destroy": ([VP], None),
+            "occu_synthesize": ([VP, P(VP), I32, VP, P(P(CsrBatch)), P(VP), P(VP)], I32),
             "occu_batch_to_device": ([VP, P(CsrBatch), P(P(CsrBatch))], I32),
             "occu_batch_free": ([P(CsrBatch)], None),
             "occu_predict": ([VP, P(CsrBatch), VP, VP, VP], I32),
@@ -152,6 +156,31 @@ def config(L=3, F_n=80, F_e=4, d=128, d_h=None, aggr=AGGR_SUM, msg=MSG_CHANNEL_S
 
 def num_params(cfg: Config) -> int:
     return int(lib().occu_num_params(C.byref(cfg)))
+
+
+class Template:
+    """A device-resident family template (occu_template, NEXT-4); freed on deletion."""
+
+    def __init__(self, model, t):
+        node_static = np.ascontiguousarray(t.node_static, dtype=np.float32)
+        node_coef = np.ascontiguousarray(t.node_coef, dtype=np.float64)
+        edge_static = np.ascontiguousarray(t.edge_static, dtype=np.float32)
+        edge_coef = np.ascontiguousarray(t.edge_coef, dtype=np.float64)
+        src = np.ascontiguousarray(t.src, dtype=np.int32)
+        dst = np.ascontiguousarray(t.dst, dtype=np.int32)
+        view = GraphView(int(t.num_nodes), len(src), src.ctypes.data_as(C.POINTER(C.c_int32)),
+                         dst.ctypes.data_as(C.POINTER(C.c_int32)))
+        self._p = C.c_void_p()
+        self.family = t.family
+        self.num_nodes, self.num_edges = int(t.num_nodes), len(src)
+        _check(lib().occu_template_create(model._ctx, C.byref(view), node_static.ctypes.data,
+                                          node_coef.ctypes.data, edge_static.ctypes.data,
+                                          edge_coef.ctypes.data, C.byref(self._p)), model._ctx)
+
+    def __del__(self):
+        if getattr(self, "_p", None) and self._p.value and _lib is not None:
+            _lib.occu_template_destroy(self._p)
+            self._p = C.c_void_p()
 
 
 class Csr:
@@ -266,6 +295,14 @@ def pack_jobs(occ, capacity=1.0):
     return slot[:n], load[:ns.value].copy()
 
 
+class _DeviceArray:
+    """Zero-copy view of library-owned device memory (__cuda_array_interface__, float32)."""
+
+    def __init__(self, ptr, shape):
+        self.__cuda_array_interface__ = {"shape": tuple(shape), "typestr": "<f4",
+                                         "data": (int(ptr or 0), False), "version": 3}
+
+
 def ctypes_view_ok() -> bool:
     return _VIEW_DT.itemsize == C.sizeof(GraphView)
 
@@ -275,6 +312,7 @@ class Model:
 
     def __init__(self, cfg: Config, device: int = 0, stream=None):
         self.cfg = cfg
+        self._device = device
         self._inflight = []
         self._ctx = C.c_void_p()
         if stream is None:
@@ -339,6 +377,29 @@ class Model:
         _check(lib().occu_load_state(self._ctx, path.encode()), self._ctx)
 
     # batches
+    # NEXT-4: on-device feature synthesis
+    def template(self, t):
+        """Upload one family template (occu_gen.templates.Template) to this ctx's device."""
+        return Template(self, t)
+
+    def synthesize(self, templates, hp):
+        """occu_synthesize: the batch of graphs templates[b] at hp[b] = (batch, cin, seq, hw),
+        built on the device.  Returns (device Csr, node_feat, edge_feat) with the features as
+        zero-copy CUDA tensors over library memory, valid until the next synthesize call."""
+        import torch
+        hp = np.ascontiguousarray(hp, dtype=np.float32).reshape(-1, 4)
+        arr = (C.c_void_p * len(templates))(*[tp._p for tp in templates])
+        out = C.POINTER(CsrBatch)()
+        nf, ef = C.c_void_p(), C.c_void_p()
+        _check(lib().occu_synthesize(self._ctx, arr, len(templates), hp.ctypes.data, C.byref(out),
+                                     C.byref(nf), C.byref(ef)), self._ctx)
+        csr = Csr(out)
+        N, E = csr.struct.num_nodes, csr.struct.num_edges
+        dev = torch.device("cuda", self._device)
+        nft = torch.as_tensor(_DeviceArray(nf.value, (N, 80)), device=dev)
+        eft = torch.as_tensor(_DeviceArray(ef.value, (E, 4)), device=dev)
+        return csr, nft, eft
+
     def to_device(self, csr: Csr) -> Csr:
         out = C.POINTER(CsrBatch)()
         _check(lib().occu_batch_to_device(self._ctx, csr._p, C.byref(out)), self._ctx)

@@ -107,3 +107,17 @@ def test_random_dag_batch():
         assert dags.is_dag(n, s, t)
         assert (s < t).all() if len(s) else True
     assert b.node_feat.shape[0] == b.num_nodes
+
+
+def test_feature_templates_exact_for_every_family():
+    """NEXT-4 templates (occu_gen/templates.py): every family's hyperparameter-dependent Table I
+    quantities are reproduced exactly (float64 ==) by the Newton form at held-out mixture
+    hyperparameters, so on-device synthesis can match the generator's features."""
+    from occu_gen import templates
+    from occu_gen.prng import Rng
+    for fam in configs.MIXTURE + ["bert_base"]:
+        t = templates.build_template(fam)
+        r = Rng(2024)
+        templates.verify(t, [configs.mixture_variant(fam, r) for _ in range(2)])
+        assert t.node_coef.shape == (t.num_nodes, 22, 12)
+        assert np.all(t.node_static[:, 42:76] == 0)
