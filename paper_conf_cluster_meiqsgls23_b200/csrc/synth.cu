@@ -66,17 +66,27 @@ __device__ __forceinline__ double poly(const double *__restrict__ c, const doubl
   return q;
 }
 
-// One CTA per graph: CSR replication with offsets, node rows, edge rows.
-__global__ void __launch_bounds__(256) synth_kernel(const SynthGraph *__restrict__ gs, int B, int N, int E,
-                                                    int32_t *node_off, int32_t *edge_off,
-                                                    int32_t *in_ptr, int32_t *out_ptr, int32_t *in_src,
-                                                    int32_t *in_dst, int32_t *in_eid, int32_t *out_pos,
-                                                    int32_t *node_graph, float *__restrict__ nf,
-                                                    float *__restrict__ ef) {
-  const int b = blockIdx.x, t = threadIdx.x;
-  const SynthGraph g = gs[b];
+// CTA (graph b, slice s): nodes [64 s, 64 s + 64) and edges [128 s, 128 s + 128) of graph b
+// (slices past the graph's end exit at once).  Phase 1: CSR replication with the graph's
+// offsets and the 22 node quantities + edge bytes (Newton form, float64) encoded into shared
+// memory; phase 2: the 64 node rows [64][80] written coalesced from the template's static
+// columns and the encoded values.
+constexpr int SN = 64, SE = 128, ST = 256;
+__global__ void __launch_bounds__(ST) synth_kernel(const SynthGraph *__restrict__ gs, int B, int N, int E,
+                                                   int32_t *node_off, int32_t *edge_off,
+                                                   int32_t *in_ptr, int32_t *out_ptr, int32_t *in_src,
+                                                   int32_t *in_dst, int32_t *in_eid, int32_t *out_pos,
+                                                   int32_t *node_graph, float *__restrict__ nf,
+                                                   float *__restrict__ ef) {
+  __shared__ float qv[SN][NQ + 5];       // encoded quantities (22), 4 x sizes (4), pad
+  __shared__ float cfgv[4];
+  const int b = blockIdx.x, sl = blockIdx.y, t = threadIdx.x;
+  const SynthGraph &g = gs[b];
+  const int n = g.n, m = g.m;
+  const int u0 = sl * SN, k0 = sl * SE;
+  if (u0 >= n && k0 >= m) return;
   const int n0 = g.node_off, e0 = g.edge_off;
-  if (t == 0) {
+  if (t == 0 && sl == 0) {
     node_off[b] = n0;
     edge_off[b] = e0;
     if (b == B - 1) {
@@ -86,41 +96,46 @@ __global__ void __launch_bounds__(256) synth_kernel(const SynthGraph *__restrict
       out_ptr[N] = E;
     }
   }
-  for (int u = t; u < g.n; u += blockDim.x) {
+  double bv[NC];
+  newton_basis(g.hp, bv);
+  const int un = max(0, min(SN, n - u0)), kn = max(0, min(SE, m - k0));
+  if (t < un) {
+    const int u = u0 + t;
     in_ptr[n0 + u] = e0 + __ldg(g.in_ptr + u);
     out_ptr[n0 + u] = e0 + __ldg(g.out_ptr + u);
     node_graph[n0 + u] = b;
   }
-  for (int k = t; k < g.m; k += blockDim.x) {
+  if (t < kn) {
+    const int k = k0 + t;
     in_src[e0 + k] = n0 + __ldg(g.in_src + k);
     in_dst[e0 + k] = n0 + __ldg(g.in_dst + k);
     in_eid[e0 + k] = e0 + __ldg(g.in_eid + k);
     out_pos[e0 + k] = e0 + __ldg(g.out_pos + k);
+    const double x = poly(g.ecoef + size_t(k) * NC, bv);
+    const size_t er = size_t(e0 + k) * FE;
+    *reinterpret_cast<float4 *>(ef + er) =
+        make_float4(__ldg(g.estatic + size_t(k) * FE), __ldg(g.estatic + size_t(k) * FE + 1), enc(x),
+                    __ldg(g.estatic + size_t(k) * FE + 3));
   }
-  double bv[NC];
-  newton_basis(g.hp, bv);
-  // node rows: element i = (u, col), coalesced over the graph's [n][80] block
-  for (int i = t; i < g.n * FN; i += blockDim.x) {
-    const int u = i / FN, c = i % FN;
+  if (t < 4) cfgv[t] = enc(double(g.hp[t]));
+  for (int i = t; i < un * NQ; i += ST) {        // the 22 quantities of the slice's nodes
+    const int r = i / NQ, q = i % NQ;
+    const double x = poly(g.ncoef + (size_t(u0 + r) * NQ + q) * NC, bv);
+    qv[r][q] = enc(x);
+    if (q >= 16 && q < 20) qv[r][NQ + (q - 16)] = enc(4.0 * x);     // bytes = 4 x size
+  }
+  __syncthreads();
+  for (int i = t; i < un * FN; i += ST) {
+    const int r = i / FN, c = i % FN;
     float v;
-    if (c >= 42 && c < 58) {
-      v = enc(poly(g.ncoef + (size_t(u) * NQ + (c - 42)) * NC, bv));          // operator hp
-    } else if (c >= 58 && c < 66) {
-      v = c < 62 ? enc(double(g.hp[c - 58])) : 0.f;                           // model config
-    } else if (c >= 66 && c < 70) {
-      v = enc(poly(g.ncoef + (size_t(u) * NQ + 16 + (c - 66)) * NC, bv));     // tensor sizes
-    } else if (c >= 70 && c < 74) {
-      v = enc(4.0 * poly(g.ncoef + (size_t(u) * NQ + 16 + (c - 70)) * NC, bv)); // bytes
-    } else if (c == 74 || c == 75) {
-      v = enc(poly(g.ncoef + (size_t(u) * NQ + 20 + (c - 74)) * NC, bv));     // FLOPs, temp
-    } else {
-      v = __ldg(g.nstatic + i);                                               // hp-independent
-    }
-    nf[size_t(n0) * FN + i] = v;
-  }
-  for (int i = t; i < g.m * FE; i += blockDim.x) {
-    const int k = i / FE, c = i % FE;
-    ef[size_t(e0) * FE + i] = c == 2 ? enc(poly(g.ecoef + size_t(k) * NC, bv)) : __ldg(g.estatic + i);
+    if (c >= 42 && c < 58) v = qv[r][c - 42];                  // operator hp
+    else if (c >= 58 && c < 62) v = cfgv[c - 58];              // model configuration
+    else if (c >= 62 && c < 66) v = 0.f;
+    else if (c >= 66 && c < 70) v = qv[r][16 + (c - 66)];      // tensor sizes
+    else if (c >= 70 && c < 74) v = qv[r][NQ + (c - 70)];      // bytes
+    else if (c == 74 || c == 75) v = qv[r][20 + (c - 74)];     // FLOPs, temp
+    else v = __ldg(g.nstatic + size_t(u0) * FN + i);           // hp-independent
+    nf[size_t(n0 + u0) * FN + i] = v;
   }
 }
 
@@ -221,6 +236,7 @@ extern "C" occu_status occu_synthesize(occu_ctx *ctx, const occu_template *const
     return fail(ctx, OCCU_EINVAL, "occu_synthesize: the templates carry Table I rows (F_n = 80, F_e = 4)");
   std::vector<SynthGraph> gs(num_graphs);
   int64_t N = 0, E = 0;
+  int slices = 1;
   for (int b = 0; b < num_graphs; ++b) {
     const occu_template *t = templates[b];
     if (!t) return fail(ctx, OCCU_EINVAL, "occu_synthesize: NULL template");
@@ -238,6 +254,7 @@ extern "C" occu_status occu_synthesize(occu_ctx *ctx, const occu_template *const
     memcpy(g.hp, hp + 4 * b, 16);
     N += t->n;
     E += t->m;
+    slices = std::max(slices, std::max((t->n + SN - 1) / SN, (t->m + SE - 1) / SE));
     if (N >= INT32_MAX || E >= INT32_MAX) return fail(ctx, OCCU_EINVAL, "occu_synthesize: N or E >= 2^31");
   }
   Workspace &w = ctx->ws;
@@ -269,7 +286,7 @@ extern "C" occu_status occu_synthesize(occu_ctx *ctx, const occu_template *const
   c->on_device = 1;
   c->priv = nullptr;          // arrays are ctx-owned (valid until the next occu_synthesize)
   OCCU_PROF_BEGIN(ctx, "synthesize", ctx->stream);
-  synth_kernel<<<num_graphs, 256, 0, ctx->stream>>>(
+  synth_kernel<<<dim3(num_graphs, slices), ST, 0, ctx->stream>>>(
       w.sdesc.as<SynthGraph>(), num_graphs, int(N), int(E), c->node_off, c->edge_off, c->in_ptr,
       c->out_ptr, c->in_src, c->in_dst, c->in_eid, c->out_pos, c->node_graph, w.snf.as<float>(),
       w.sef.as<float>());
