@@ -455,6 +455,25 @@ def main():
                     "kernel_ms_per_step": {k: v["ms_per_step"] for k, v in kr.items()}, "kernels": kr,
                     "what": "ANEE reading B: per-channel softmax over each destination's in-edges"}
         del mr
+        # reading B in OCCU_BF16 (R40): BF16 logits / h̄ / e' / h, FP32 softmax and sums
+        mrb = occu.Model(occu.config(L=3, F_n=80, F_e=4, d=128, msg=occu.MSG_NEIGHBOR_SOFTMAX,
+                                     prec=occu.BF16), device=local, stream=stream.cuda_stream)
+        mrb.init_weights(42)
+        inferrb = lambda: mrb.predict(csr, nf, ef, outr)
+        timed(inferrb, args.warmup, mdl=mrb)
+        bar()
+        trb, lrb = timed(inferrb, args.steps, mdl=mrb)
+        bar()
+        timed(inferrb, args.steps, profile=True, mdl=mrb)
+        bar()
+        msrb = max_over_ranks(float(np.sum(trb)) / args.steps)
+        algrb = algorithmic_bytes(N, E, B, d, rrows=rrows, sa=2)
+        algrb["gather_segsoftmax"] = algrb["gather_segsum"]
+        krb, roofrb = kernel_table(mrb.profile(), algrb, {})
+        readingb["bf16"] = {"value": B * world / (msrb * 1e-3), "unit": "graphs/s", "ms_per_step": msrb,
+                            "dtype": "bf16", "tolerance": 1e-2, "gpu_launches": lrb, "roofline": roofrb,
+                            "kernel_ms_per_step": {k: v["ms_per_step"] for k, v in krb.items()}}
+        del mrb
 
     # ---- NEXT-2: Set-Transformer decoder readout (k = 4 seeds, 4 heads), inference, same batch
     decoder = None

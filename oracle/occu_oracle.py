@@ -291,9 +291,18 @@ def forward_bf16(params, cfg, pk, node_feat, edge_feat, rnd=None):
         tensor_core = not (i == 0 and e.shape[1] <= 16)
         z = (r16(e) @ r16(W_e).T) if tensor_core else (e @ W_e.T)   # P145
         e_new = r16(sigmoid(alpha[:, None] * z))                  # stored BF16
-        v = e_new @ r16(W_m).T                                    # P149
-        g = r16(softmax_channels(v))                              # stored BF16 (R24)
-        A = segment_sum(g * hbar[s_k], t_k, N)                    # P149 (R4, reading A)
+        if cfg.get("msg", MSG_CHANNEL_SOFTMAX) == MSG_CHANNEL_SOFTMAX:
+            v = e_new @ r16(W_m).T                                # P149
+            g = r16(softmax_channels(v))                          # stored BF16 (R24)
+        else:
+            # reading B (NEXT-1) in OCCU_BF16 (R40): the logits are stored BF16; the softmax
+            # over the destination's in-edges and its weights stay unrounded
+            v = r16(e_new @ r16(W_m).T)
+            M = np.full((N, v.shape[1]), -np.inf)
+            np.maximum.at(M, t_k, v)
+            ex = np.exp(v - M[t_k])
+            g = ex / segment_sum(ex, t_k, N)[t_k]
+        A = segment_sum(g * hbar[s_k], t_k, N)                    # P149 (R4)
         if cfg["aggr"] == AGGR_MEAN:
             A = A / np.maximum(deg, 1)[:, None]
         h_f = leaky_relu(A, slope)

@@ -36,7 +36,7 @@ namespace {
 constexpr int TM = 128;
 constexpr int NTH = 832;
 constexpr int EPI0 = 10;
-constexpr int EPI_NODE = 0, EPI_EDGE = 1, EPI_GATE = 2, EPI_EDGEBWD = 5;
+constexpr int EPI_NODE = 0, EPI_EDGE = 1, EPI_GATE = 2, EPI_LOGIT = 3, EPI_EDGEBWD = 5;
 constexpr float LOG2E = 1.4426950408889634f;
 
 __device__ __forceinline__ float lrelu(float x, float s) { return x > 0.f ? x : s * x; }
@@ -336,6 +336,17 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_bf16_kernel(const __grid_const
           for (int u = 0; u < 16; ++u) o[u] = fast_rcp(1.f + ex2(__uint_as_float(r[u]) * cexp));  // e' (R2, R3)
           warp_store_bf16(wbuf, a.out, wrow0, wrows, cb + c0, D, o, lane);
         }
+      } else if (EPI == EPI_LOGIT) {      // reading B: the logits v = W_m e' -> BF16
+#pragma unroll 1
+        for (int c0 = 0; c0 < DH; c0 += 16) {
+          uint32_t r[16];
+          tc::tmem_ld16(acc + c0, r);
+          tc::tmem_ld_wait();
+          float o[16];
+#pragma unroll
+          for (int u = 0; u < 16; ++u) o[u] = __uint_as_float(r[u]);
+          warp_store_bf16(wbuf, a.out, wrow0, wrows, cb + c0, D, o, lane);
+        }
       } else if (EPI == EPI_EDGEBWD) {
         const float cexp = al * LOG2E;
         double dpart = 0.0;                       // dα = <dy, z> in float64 (cancellation)
@@ -588,8 +599,16 @@ int forward_layer_bf16(const occu_ctx *ctx, const DevCsr &csr, int layer, const 
     rg.rev = ctx->l2_order;
     rg.K = D; rg.R = csr.E; rg.out = reinterpret_cast<__nv_bfloat16 *>(a.g);
     rg.wimg = tc_wimg(ctx, 2, layer); rg.wf = tc_wfexp(ctx, 2, layer);
-    if ((r = launch_bf<D, EPI_GATE, false>(ctx, rg, a.e_out, "gate_tc", st)) < 0) return r;
+    if (ctx->cfg.msg == OCCU_MSG_NEIGHBOR_SOFTMAX) {       // reading B: logits, then the
+      if ((r = launch_bf<D, EPI_LOGIT, false>(ctx, rg, a.e_out, "gate_tc", st)) < 0) return r;
+    } else if ((r = launch_bf<D, EPI_GATE, false>(ctx, rg, a.e_out, "gate_tc", st)) < 0) {
+      return r;
+    }
     n += r;
+  }
+  if (ctx->cfg.msg == OCCU_MSG_NEIGHBOR_SOFTMAX) {          // segmented softmax over in-edges
+    if ((r = launch_gather_segsoftmax_bf16(ctx, csr, a.g, a.hbar, a.h_out, a.rpart, a.save_w, st)) < 0) return r;
+    return n + r;
   }
   if ((r = launch_gather_segsum_bf16(ctx, csr, a.g, a.hbar, a.h_out, a.rpart, st)) < 0) return r;
   return n + r;

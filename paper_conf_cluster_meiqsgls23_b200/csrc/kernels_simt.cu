@@ -713,10 +713,11 @@ __global__ void __launch_bounds__(NT) gate_bwd_stream_kernel(
 // overwrites v_k with w_k (the weights the backward reads; each row is read before it is
 // written and only by its owner warp).  RP: last layer, readout chunk partials as v2.
 // ---------------------------------------------------------------------------
-template <int D, int G, bool RP, bool W>
+// BF (OCCU_BF16): v, h̄ and h are BF16 rows (the softmax, the sums and the readout stay FP32).
+template <int D, int G, bool RP, bool W, bool BF>
 __global__ void __launch_bounds__(NT) gather_segsoftmax_kernel(
-    float *__restrict__ v, const float *__restrict__ hbar, const int32_t *__restrict__ in_ptr,
-    const int32_t *__restrict__ in_src, int N, int mean, float slope, float *__restrict__ h_out,
+    void *__restrict__ v, const void *__restrict__ hbar, const int32_t *__restrict__ in_ptr,
+    const int32_t *__restrict__ in_src, int N, int mean, float slope, void *__restrict__ h_out,
     const int32_t *__restrict__ node_graph, float *__restrict__ rpart) {
   constexpr int V = D / 32;
   constexpr int NPW = 8;
@@ -755,10 +756,10 @@ __global__ void __launch_bounds__(NT) gather_segsoftmax_kernel(
         for (int c = 0; c < V; ++c) inv[c] = 1.f / sum[c];
         for (int k = seg_beg; k < seg_end; ++k) {
           float x[V];
-          load_row<V, false>(v, long(k), D, lane, x);
+          load_row<V, BF>(v, long(k), D, lane, x);
 #pragma unroll
           for (int c = 0; c < V; ++c) x[c] = ex2f_fast((x[c] - m[c]) * L2E) * inv[c];
-          store_row<V>(v + long(k) * D + lane * V, x);
+          store_row_t<V, BF>(v, long(k), D, lane, x);
         }
       }
 #pragma unroll
@@ -766,7 +767,7 @@ __global__ void __launch_bounds__(NT) gather_segsoftmax_kernel(
         m[c] = -INFINITY;
         sum[c] = acc[c] = 0.f;
       }
-      if (!RP || h_out) store_row_t<V, false>(h_out, t0 + nd, D, lane, o);
+      if (!RP || h_out) store_row_t<V, BF>(h_out, t0 + nd, D, lane, o);
       if (RP) {
         const int gc = __shfl_sync(0xffffffffu, gr_l, nd);
         const int gn = __shfl_sync(0xffffffffu, gr_l, (nd + 1) & 31);
@@ -783,7 +784,7 @@ __global__ void __launch_bounds__(NT) gather_segsoftmax_kernel(
       const int cnt = min(32, e_end - base);
       const int s_l = lane < cnt ? __ldg(in_src + base + lane) : 0;
       for (int j = 0; j < cnt; j += G) {
-        RawRow<V, false> vr[G], hr[G];
+        RawRow<V, BF> vr[G], hr[G];
 #pragma unroll
         for (int u = 0; u < G; ++u) {
           const int kk = min(j + u, cnt - 1);
@@ -1714,20 +1715,20 @@ static int gather_bf16_impl(const occu_ctx *ctx, const DevCsr &csr, const void *
   return 1;
 }
 
-template <int D>
-static int segsoftmax_impl(const occu_ctx *ctx, const DevCsr &csr, float *v, const float *hbar,
-                           float *h_out, float *rpart, bool write_w, cudaStream_t st) {
+template <int D, bool BF>
+static int segsoftmax_impl(const occu_ctx *ctx, const DevCsr &csr, void *v, const void *hbar,
+                           void *h_out, float *rpart, bool write_w, cudaStream_t st) {
   if (csr.N <= 0) return 0;
   const int mean = ctx->cfg.aggr == OCCU_AGGR_MEAN;
   const int grid = grid_for(long(csr.N) * 4, NT, 8 * ctx->num_sms);
   OCCU_PROF_BEGIN(ctx, "gather_segsoftmax", st);
 #define OCCU_GS_ARGS v, hbar, csr.in_ptr, csr.in_src, csr.N, mean, ctx->cfg.slope, h_out, csr.node_graph, rpart
   if (write_w) {
-    if (rpart) launch_pdl(ctx->pdl & 2, gather_segsoftmax_kernel<D, 4, true, true>, grid, NT, 0, st, OCCU_GS_ARGS);
-    else launch_pdl(ctx->pdl & 2, gather_segsoftmax_kernel<D, 4, false, true>, grid, NT, 0, st, OCCU_GS_ARGS);
+    if (rpart) launch_pdl(ctx->pdl & 2, gather_segsoftmax_kernel<D, 4, true, true, BF>, grid, NT, 0, st, OCCU_GS_ARGS);
+    else launch_pdl(ctx->pdl & 2, gather_segsoftmax_kernel<D, 4, false, true, BF>, grid, NT, 0, st, OCCU_GS_ARGS);
   } else {
-    if (rpart) launch_pdl(ctx->pdl & 2, gather_segsoftmax_kernel<D, 4, true, false>, grid, NT, 0, st, OCCU_GS_ARGS);
-    else launch_pdl(ctx->pdl & 2, gather_segsoftmax_kernel<D, 4, false, false>, grid, NT, 0, st, OCCU_GS_ARGS);
+    if (rpart) launch_pdl(ctx->pdl & 2, gather_segsoftmax_kernel<D, 4, true, false, BF>, grid, NT, 0, st, OCCU_GS_ARGS);
+    else launch_pdl(ctx->pdl & 2, gather_segsoftmax_kernel<D, 4, false, false, BF>, grid, NT, 0, st, OCCU_GS_ARGS);
   }
 #undef OCCU_GS_ARGS
   OCCU_PROF_END(ctx);
@@ -1738,8 +1739,18 @@ static int segsoftmax_impl(const occu_ctx *ctx, const DevCsr &csr, float *v, con
 int launch_gather_segsoftmax(const occu_ctx *ctx, const DevCsr &csr, float *v, const float *hbar,
                              float *h_out, float *rpart, bool write_w, cudaStream_t st) {
   switch (ctx->cfg.d) {
-    case 64: return segsoftmax_impl<64>(ctx, csr, v, hbar, h_out, rpart, write_w, st);
-    case 128: return segsoftmax_impl<128>(ctx, csr, v, hbar, h_out, rpart, write_w, st);
+    case 64: return segsoftmax_impl<64, false>(ctx, csr, v, hbar, h_out, rpart, write_w, st);
+    case 128: return segsoftmax_impl<128, false>(ctx, csr, v, hbar, h_out, rpart, write_w, st);
+    default: return -int(cudaErrorInvalidValue);
+  }
+}
+
+// OCCU_BF16 reading B: BF16 logits / weights v, h̄ and h
+int launch_gather_segsoftmax_bf16(const occu_ctx *ctx, const DevCsr &csr, void *v, const void *hbar,
+                                  void *h_out, float *rpart, bool write_w, cudaStream_t st) {
+  switch (ctx->cfg.d) {
+    case 64: return segsoftmax_impl<64, true>(ctx, csr, v, hbar, h_out, rpart, write_w, st);
+    case 128: return segsoftmax_impl<128, true>(ctx, csr, v, hbar, h_out, rpart, write_w, st);
     default: return -int(cudaErrorInvalidValue);
   }
 }

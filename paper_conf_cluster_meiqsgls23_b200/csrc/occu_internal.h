@@ -221,6 +221,8 @@ int launch_gather_segsum(const occu_ctx *ctx, const DevCsr &csr, const float *g,
 int launch_gather_segsoftmax(const occu_ctx *ctx, const DevCsr &csr, float *v, const float *hbar,
                              float *h_out, float *rpart, bool write_w, cudaStream_t st);
 // OCCU_BF16: g, h̄, h stored as BF16 (FP32 arithmetic); rpart stays FP32.
+int launch_gather_segsoftmax_bf16(const occu_ctx *ctx, const DevCsr &csr, void *v, const void *hbar,
+                                  void *h_out, float *rpart, bool write_w, cudaStream_t st);
 int launch_gather_segsum_bf16(const occu_ctx *ctx, const DevCsr &csr, const void *g,
                               const void *hbar, void *h_out, float *rpart, cudaStream_t st);
 // OCCU_BF16 forward layer (kernels_bf16.cu); FwdLayerArgs pointers to h̄, e', g, h hold BF16.

@@ -157,8 +157,8 @@ occu_status validate_cfg(const occu_config *c) {
     return fail(nullptr, OCCU_EINVAL, "aggr must be SUM or MEAN");
   if (c->msg != OCCU_MSG_CHANNEL_SOFTMAX && c->msg != OCCU_MSG_NEIGHBOR_SOFTMAX)
     return fail(nullptr, OCCU_EINVAL, "msg must be CHANNEL_SOFTMAX (reading A) or NEIGHBOR_SOFTMAX (reading B)");
-  if (c->msg == OCCU_MSG_NEIGHBOR_SOFTMAX && (c->prec != OCCU_FP32 || c->F_n > 128))
-    return fail(nullptr, OCCU_EINVAL, "reading B (NEIGHBOR_SOFTMAX) runs in OCCU_FP32 on the tensor-core path (F_n <= 128)");
+  if (c->msg == OCCU_MSG_NEIGHBOR_SOFTMAX && c->F_n > 128)
+    return fail(nullptr, OCCU_EINVAL, "reading B (NEIGHBOR_SOFTMAX) runs on the tensor-core path (F_n <= 128)");
   if (c->prec != OCCU_FP32 && c->prec != OCCU_BF16)
     return fail(nullptr, OCCU_EINVAL, "prec must be OCCU_FP32 or OCCU_BF16");
   if (c->prec == OCCU_BF16 && !(c->F_n <= 128 && (c->F_e <= 16 || c->F_e % 64 == 0)))
@@ -397,6 +397,8 @@ occu_status grads_impl(occu_ctx *ctx, const occu_batch *batch, const float *targ
     return fail(ctx, OCCU_EINVAL, "the Set-Transformer decoder readout is inference-only in this build");
   if (ctx->cfg.graphormer > 0)
     return fail(ctx, OCCU_EINVAL, "Graphormer layers are inference-only in this build");
+  if (ctx->cfg.msg == OCCU_MSG_NEIGHBOR_SOFTMAX && ctx->cfg.prec == OCCU_BF16)
+    return fail(ctx, OCCU_EINVAL, "reading B in OCCU_BF16 is inference-only in this build");
   ctx->launches = 0;
   if ((st = resolve_csr(ctx, batch->csr, csr)) != OCCU_OK) return st;
   if ((st = stage_inputs(ctx, csr, batch->node_feat, batch->edge_feat, targets, stg)) != OCCU_OK)

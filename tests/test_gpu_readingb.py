@@ -148,8 +148,77 @@ def test_readingb_training_trajectory():
 
 
 def test_readingb_errors():
+    occu.Model(occu.config(L=2, d=64, msg=MSGB, prec=occu.BF16))      # valid since R40 (inference)
     with pytest.raises(occu.OccuError):
-        occu.Model(occu.config(L=2, d=64, msg=MSGB, prec=occu.BF16))
+        occu.Model(occu.config(L=2, F_n=200, d=64, msg=MSGB))
     m = occu.Model(mk(2, 64))
     with pytest.raises(occu.OccuError):
         m.set_kernel_path(1)
+
+
+# ------------------------------------------ reading B in OCCU_BF16 (R40), inference
+def _mkb(L, d, aggr=0):
+    return occu.config(L=L, F_n=80, F_e=4, d=d, aggr=aggr, prec=occu.BF16,
+                       msg=occu.MSG_NEIGHBOR_SOFTMAX)
+
+
+def _ocfgb(c):
+    return dict(L=c.L, F_n=c.F_n, F_e=c.F_e, d=c.d, d_h=c.d_h, aggr=c.aggr, msg=c.msg,
+                slope=float(np.float32(c.slope)))
+
+
+def _wcfgb(c):
+    return weights.ModelConfig(L=c.L, F_n=c.F_n, F_e=c.F_e, d=c.d, d_h=c.d_h, aggr=c.aggr, msg=c.msg)
+
+
+def _relb(a, b):
+    a = np.asarray(a, np.float64)
+    b = np.asarray(b, np.float64)
+    nb = np.linalg.norm(b)
+    return np.linalg.norm(a - b) / (nb if nb > 0 else 1.0)
+
+
+@pytest.mark.parametrize("L,d,aggr,seed", [(2, 64, 0, 1), (3, 128, 0, 2), (3, 128, 1, 3)])
+def test_readingb_bf16_intermediates_and_predictions(L, d, aggr, seed):
+    """Every intermediate vs oracle.forward_bf16 (the mode's roundings in float64) at 3e-3,
+    ŷ vs the float64 oracle at the BF16 criterion (rel-L2 <= 1e-2, per graph
+    1e-2·max(|ŷ|, 0.1), R25)."""
+    c = _mkb(L, d, aggr)
+    b = configs.random_dag_batch(40, 700 + seed, max_nodes=60, hub=True)
+    flat = weights.init_flat(_wcfgb(c), seed)
+    m = occu.Model(c)
+    m.set_params(flat)
+    m.keep_intermediates(True)
+    y = m.predict(occu.pack(b.graphs), b.node_feat, b.edge_feat)
+    params = oracle.unflatten(_ocfgb(c), flat.astype(np.float64))
+    pk = oracle.pack(b.graphs)
+    emu = oracle.forward_bf16(params, _ocfgb(c), pk, b.node_feat, b.edge_feat)
+    ref = oracle.forward(params, _ocfgb(c), pk, b.node_feat, b.edge_feat)
+    N, E, B = pk["num_nodes"], pk["num_edges"], pk["num_graphs"]
+    for i in range(L):
+        lay = emu["layers"][i]
+        assert _relb(m.get_tensor(occu.T_HBAR, i, (N, d)), lay["hbar"]) <= 3e-3, ("hbar", i)
+        assert _relb(m.get_tensor(occu.T_E, i, (E, d)), lay["e"]) <= 3e-3, ("e", i)
+        assert _relb(m.get_tensor(occu.T_H, i, (N, d)), lay["h"]) <= 3e-3, ("h", i)
+    assert _relb(m.get_tensor(occu.T_R, 0, (B, d)), emu["r"]) <= 3e-3
+    yr = ref["yhat"]
+    assert _relb(y, yr) <= 1e-2
+    assert np.all(np.abs(y - yr) <= 1e-2 * np.maximum(np.abs(yr), 0.1)), np.abs(y - yr).max()
+
+
+def test_readingb_bf16_cfg2_sampled_and_training_rejected():
+    c = _mkb(3, 128)
+    b = configs.cfg2(256)
+    flat = weights.init_flat(_wcfgb(c), 42)
+    m = occu.Model(c)
+    m.set_params(flat)
+    csr = occu.pack(b.graphs)
+    y1 = m.predict(csr, b.node_feat, b.edge_feat)
+    assert np.array_equal(y1, m.predict(csr, b.node_feat, b.edge_feat))
+    params = oracle.unflatten(_ocfgb(c), flat.astype(np.float64))
+    for gi in (0, 131, 255):
+        s = b.subset([gi])
+        yr = oracle.predict(params, _ocfgb(c), s.graphs, s.node_feat, s.edge_feat)
+        assert abs(y1[gi] - yr[0]) <= 1e-2 * max(abs(yr[0]), 0.1), gi
+    with pytest.raises(occu.OccuError):
+        m.train_step(csr, b.node_feat, b.edge_feat, b.targets, 1e-4)

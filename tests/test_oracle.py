@@ -831,3 +831,30 @@ def test_occu_packing_invariants_and_bounds():
     assert np.array_equal(a, np.repeat(np.arange(3), 4))
     a, _ = oracle.occu_packing(np.array([-0.1, 1.3, 0.2], np.float32))   # clamp, oversize alone
     assert np.array_equal(a, [0, 1, 0])
+
+
+def test_forward_bf16_reading_b_identity_rounding_and_chain_closed_form():
+    """Reading B in OCCU_BF16 (R40): with the rounding replaced by the identity, forward_bf16
+    is forward() (same steps); with BF16 rounding, a single in-edge still gives weight
+    exactly 1 (softmax over one edge), so a chain's h_t = LReLU(h̄_src) holds per layer
+    with the BF16-stored h̄."""
+    cfg = cfg_dict(L=2, F_n=80, F_e=4, d=16, d_h=8)
+    cfg["msg"] = 1
+    b = configs.random_dag_batch(5, 91, max_nodes=20, hub=True)
+    wc = weights.ModelConfig(L=2, F_n=80, F_e=4, d=16, d_h=8, msg=1)
+    p = oracle.unflatten(cfg, weights.init_flat(wc, 3).astype(np.float64))
+    pk = oracle.pack(b.graphs)
+    f = oracle.forward(p, cfg, pk, b.node_feat, b.edge_feat)
+    fb = oracle.forward_bf16(p, cfg, pk, b.node_feat, b.edge_feat, rnd=lambda x: np.asarray(x, np.float64))
+    assert np.allclose(fb["yhat"], f["yhat"], rtol=1e-12, atol=1e-14)
+    for i in range(2):
+        assert np.allclose(fb["layers"][i]["g"], f["layers"][i]["g"], rtol=1e-12, atol=1e-14)
+    chain = [(6, np.arange(5, dtype=np.int32), np.arange(1, 6, dtype=np.int32))]
+    nf = np.random.default_rng(1).random((6, 80))
+    ef = np.random.default_rng(2).random((5, 4))
+    pkc = oracle.pack(chain)
+    fc = oracle.forward_bf16(p, cfg, pkc, nf, ef)
+    for i in range(2):
+        lay = fc["layers"][i]
+        assert np.array_equal(lay["g"], np.ones_like(lay["g"]))
+        assert np.allclose(lay["h_f32"][1:], oracle.leaky_relu(lay["hbar"][:5], cfg["slope"]), rtol=1e-15, atol=0)
