@@ -600,6 +600,36 @@ def main():
            "h2d_bytes_per_step": int(batch.node_feat.nbytes + batch.edge_feat.nbytes + csr_bytes),
            "d2h_bytes_per_step": int(B * 4),
            "includes": "per step: occu_pack (host C++, from concatenated edge lists) + occu_predict_async with pinned host buffers (H2D on the copy stream, kernels, D2H of the predictions), pipelined across steps; timed to occu_wait"}
+    # the same CFG2 step with the inputs given as (template, hyperparameters) per graph and the
+    # features / CSR synthesized on the device (NEXT-4): H2D 112 B per graph
+    if args.path == 0:
+        from occu_gen import templates as tmpl_mod
+        t_r50 = model.template(tmpl_mod.build_template("resnet50"))
+        grid = configs.cnn_grid()
+        hp2 = np.stack([tmpl_mod.hp_vector("resnet50", grid[i % len(grid)]) for i in range(B)]).astype(np.float32)
+        tl2 = [t_r50] * B
+        d_o2 = torch.empty(B, dtype=torch.float32, device=dev)
+        pin_o2 = torch.empty(B, dtype=torch.float32).pin_memory()
+
+        def e2e_synth2():
+            c_, n_, e_ = model.synthesize(tl2, hp2)
+            model.predict(c_, n_, e_, d_o2)
+            pin_o2.copy_(d_o2)
+        for _ in range(args.warmup):
+            e2e_synth2()
+        torch.cuda.synchronize()
+        bar()
+        t0 = time.perf_counter()
+        for _ in range(args.steps):
+            e2e_synth2()
+        torch.cuda.synchronize()
+        ms_s2 = max_over_ranks((time.perf_counter() - t0) * 1e3 / args.steps)
+        e2e["synthesized"] = {"value": B * world / (ms_s2 * 1e-3), "unit": "graphs/s", "ms_per_step": ms_s2,
+                              "h2d_bytes_per_step": int(B * 112), "d2h_bytes_per_step": int(B * 4),
+                              "includes": "per step: occu_synthesize from (ResNet-50 template, batch, cin) "
+                                          "per graph (CSR + Table I rows built on the GPU) + occu_predict "
+                                          "+ D2H of the predictions, blocking"}
+        del t_r50, tl2
 
     # ---- training step (DP over graphs, NCCL allreduce inside the library when N > 1)
     train = None
