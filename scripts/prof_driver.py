@@ -17,6 +17,7 @@ ap.add_argument("--graphs", type=int, default=256)
 ap.add_argument("--bf16", action="store_true")
 ap.add_argument("--graphormer", type=int, default=0)
 ap.add_argument("--decoder", action="store_true")
+ap.add_argument("--synth", action="store_true", help="inputs synthesized on the device (NEXT-4)")
 a = ap.parse_args()
 dev = torch.device("cuda", 0)
 m = occu.Model(occu.config(L=3, F_n=80, F_e=4, d=128, prec=occu.BF16 if a.bf16 else occu.FP32,
@@ -29,7 +30,15 @@ csr = m.to_device(occu.pack(b.graphs))
 nf = torch.from_numpy(b.node_feat).to(dev)
 ef = torch.from_numpy(b.edge_feat).to(dev)
 yt = torch.from_numpy(b.targets).to(dev)
+if a.synth:
+    import numpy as np
+    from occu_gen import templates
+    t = m.template(templates.build_template("resnet50"))
+    grid = configs.cnn_grid()
+    hp = np.stack([templates.hp_vector("resnet50", grid[i % len(grid)]) for i in range(a.graphs)]).astype(np.float32)
 for _ in range(a.steps):
+    if a.synth:
+        csr, nf, ef = m.synthesize([t] * a.graphs, hp)
     if a.train:
         m.train_step(csr, nf, ef, yt, 1e-4, want_loss=False)
     else:

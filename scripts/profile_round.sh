@@ -19,13 +19,13 @@ timeout 900 ncu --set full --clock-control none --import-source on \
   python scripts/prof_driver.py --steps 2 --bf16 > gpurun_out/prof_bf16.log 2>&1
 echo "bf16 rc=$?" >> gpurun_out/prof_bf16.log
 timeout 900 ncu --set full --clock-control none --import-source on \
-  -k regex:"gph_|set_decoder" -s 8 -c 8 -o gpurun_out/prof_next \
-  python scripts/prof_driver.py --steps 2 --graphormer 2 --decoder > gpurun_out/prof_next.log 2>&1
+  -k regex:"gph_|set_decoder|synth" -s 10 -c 9 -o gpurun_out/prof_next \
+  python scripts/prof_driver.py --steps 2 --graphormer 2 --decoder --synth > gpurun_out/prof_next.log 2>&1
 echo "next rc=$?" >> gpurun_out/prof_next.log
 # summarise on the box (the .ncu-rep files are too big to bring back whole)
 PROFILES_OUT=gpurun_out/profiles_new python scripts/summarize_ncu.py ${TAG:-r01} > gpurun_out/summarize.log 2>&1
 for f in gpurun_out/prof_*.ncu-rep; do
-  python scripts/ncu_stalls.py "$f" "gph_attn|gather_segsum|set_decoder" 30 > "${f%.ncu-rep}_stalls.txt" 2>&1
+  python scripts/ncu_stalls.py "$f" "gph_attn|gather_segsum|set_decoder|synth" 30 > "${f%.ncu-rep}_stalls.txt" 2>&1
 done
 du -sh gpurun_out/* > gpurun_out/sizes.txt
 rm -f gpurun_out/prof_full.ncu-rep gpurun_out/prof_train.ncu-rep gpurun_out/prof_bf16.ncu-rep

@@ -10,7 +10,8 @@ def kname(full):
     if m:
         return ["node_tc", "edge_tc", "gate_tc", "plain_tc", "gatebwd_tc", "edgebwd_tc",
                 "gateagg_tc"][int(m.group(2))]
-    for k, v in [("gph_attn", "gph_attn"), ("gph_ln", "gph_ln"), ("set_decoder_prep", "set_decoder_prep"),
+    for k, v in [("synth_kernel", "synthesize"), ("set_decoder_pool", "set_decoder_pool"),
+                 ("gph_attn", "gph_attn"), ("gph_ln", "gph_ln"), ("set_decoder_prep", "set_decoder_prep"),
                  ("set_decoder_kernel", "set_decoder"), ("gather_segsoftmax", "gather_segsoftmax"),
                  ("edgegate", "edge_gate_tc"), ("edge_small", "edge_small"), ("wgrad_tc", "wgrad_tc"), ("wimage", "wimage"),
                  ("split_reduce", "split_reduce"), ("agg_fixup", "agg_fixup"),
@@ -104,7 +105,7 @@ if traffic_bf:
     json.dump(traffic_bf, open(os.path.join(out, "traffic_bf16.json"), "w"), indent=1)
 with open(os.path.join(out, f"{tag}_ncu_summary.md"), "w") as f:
   for title, traffic in (("OCCU_FP32 (inference + training)", traffic), ("OCCU_BF16 inference", traffic_bf),
-                         ("NEXT-2/3 kernels: Graphormer x2 + decoder readout, OCCU_FP32 inference", traffic_nx)):
+                         ("NEXT-2/3/4 kernels: Graphormer x2 + decoder readout + on-device synthesis, OCCU_FP32 inference", traffic_nx)):
     if not traffic:
         continue
     f.write(f"# {tag}: ncu --set full --clock-control none (serialised, cold-cache replays), {title}\n\n")
