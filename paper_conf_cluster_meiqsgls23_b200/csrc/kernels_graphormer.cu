@@ -586,7 +586,7 @@ __device__ __forceinline__ void fence_proxy_async_smem() {
   asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
 }
 
-__global__ void __launch_bounds__(128) gph_attn_tc_kernel(const AttnArgs a) {
+__global__ void __launch_bounds__(128, 4) gph_attn_tc_kernel(const AttnArgs a) {
   using namespace gtc;
   extern __shared__ __align__(1024) uint8_t gsm_raw[];
   uint8_t *sm = gsm_raw + ((1024u - (tc::smem_u32(gsm_raw) & 1023u)) & 1023u);
@@ -701,37 +701,36 @@ __global__ void __launch_bounds__(128) gph_attn_tc_kernel(const AttnArgs a) {
       tc::tmem_ld32(lane_base + SC, s0);
       tc::tmem_ld32(lane_base + SC + 32, s1);
       tc::tmem_ld_wait();
-      float sv[64];
       float bm = -INFINITY;
-      if (__all_sync(0xffffffffu, kb >= lo && kb + KB <= hi)) {    // block inside every row's graph
+      if (!__all_sync(0xffffffffu, kb >= lo && kb + KB <= hi)) {   // mask keys outside the row's graph
 #pragma unroll
-        for (int j = 0; j < 64; ++j) {
-          sv[j] = __uint_as_float(j < 32 ? s0[j] : s1[j - 32]);
-          bm = fmaxf(bm, sv[j]);
-        }
-      } else {
-#pragma unroll
-        for (int j = 0; j < 64; ++j) {
-          const float x = __uint_as_float(j < 32 ? s0[j] : s1[j - 32]);
-          const int key = kb + j;
-          sv[j] = (key >= lo && key < hi) ? x : -INFINITY;
-          bm = fmaxf(bm, sv[j]);
+        for (int j = 0; j < 32; ++j) {
+          if (!(kb + j >= lo && kb + j < hi)) s0[j] = __float_as_uint(-INFINITY);
+          if (!(kb + 32 + j >= lo && kb + 32 + j < hi)) s1[j] = __float_as_uint(-INFINITY);
         }
       }
+#pragma unroll
+      for (int j = 0; j < 32; ++j) bm = fmaxf(bm, fmaxf(__uint_as_float(s0[j]), __uint_as_float(s1[j])));
       const float mn = fmaxf(m, bm);
       const float ref = mn == -INFINITY ? 0.f : mn;
       const float f = ex2f(m - ref);
       m = mn;
       float sum = 0.f;
 #pragma unroll
-      for (int j = 0; j < 32; ++j) {
-        const float p0 = ex2f(sv[2 * j] - ref), p1 = ex2f(sv[2 * j + 1] - ref);
-        sum += p0 + p1;
-        split_h2(p0, p1, s0[j], s1[j]);
+      for (int hf = 0; hf < 2; ++hf) {         // P in two 16-column halves (fewer live registers)
+        uint32_t ph[16], pl[16];
+#pragma unroll
+        for (int j = 0; j < 16; ++j) {
+          const uint32_t *src = hf == 0 ? s0 : s1;
+          const float p0 = ex2f(__uint_as_float(src[2 * j]) - ref);
+          const float p1 = ex2f(__uint_as_float(src[2 * j + 1]) - ref);
+          sum += p0 + p1;
+          split_h2(p0, p1, ph[j], pl[j]);
+        }
+        tc::tmem_st16(lane_base + PH + 16 * hf, ph);
+        tc::tmem_st16(lane_base + PL + 16 * hf, pl);
       }
       l = l * f + sum;
-      tc::tmem_st32(lane_base + PH, s0);
-      tc::tmem_st32(lane_base + PL, s1);
       if (__any_sync(0xffffffffu, f != 1.f)) {     // rescale the O row (warp-collective)
         uint32_t o[32];
         tc::tmem_ld32(lane_base + OC, o);
