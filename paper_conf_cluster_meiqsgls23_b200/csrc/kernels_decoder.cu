@@ -15,8 +15,10 @@
 //    vectors only.  Fixed order everywhere (deterministic).
 //  * The rest (W_v, W_o, LayerNorms, the k-element SAB, the FFNs, the head) is k-vector work
 //    per graph: warp-per-output-row GEMVs against L2-resident weights, one CTA per graph.
+#include <cuda_fp16.h>
 #include <cuda_runtime.h>
 #include <math.h>
+#include <stdlib.h>
 #include <stdint.h>
 
 #include "occu_internal.h"
@@ -333,6 +335,192 @@ __global__ void __launch_bounds__(DT) set_decoder_pool_kernel(const DecArgs a, c
   }
 }
 
+// Pool on the legacy tensor path (mma.sync m16n8k16, fp16x2 3-product split = FP32 accuracy):
+// per 32-row chunk of Z, the scores S[32][16] = Z·M (4 warps, one 16x8 tile each, K = D) and
+// the weighted sums P[16][D] += W[16][32]·Z[32][D] (8 warps, D/64 n-tile pairs each); the
+// online softmax bookkeeping (per (seed, head) column over the chunk's rows) stays on CUDA cores.
+__device__ __forceinline__ void dsplit_h2(float x0, float x1, uint32_t &hi, uint32_t &lo) {
+  const __half2 h = __floats2half2_rn(x0, x1);
+  const float2 hf = __half22float2(h);
+  const __half2 l = __floats2half2_rn(x0 - hf.x, x1 - hf.y);
+  hi = *reinterpret_cast<const uint32_t *>(&h);
+  lo = *reinterpret_cast<const uint32_t *>(&l);
+}
+__device__ __forceinline__ void dmma(float (&c)[4], const uint32_t (&a)[4], uint32_t b0, uint32_t b1) {
+  asm volatile(
+      "mma.sync.aligned.m16n8k16.row.col.f32.f16.f16.f32 {%0,%1,%2,%3}, {%4,%5,%6,%7}, {%8,%9}, "
+      "{%0,%1,%2,%3};"
+      : "+f"(c[0]), "+f"(c[1]), "+f"(c[2]), "+f"(c[3])
+      : "r"(a[0]), "r"(a[1]), "r"(a[2]), "r"(a[3]), "r"(b0), "r"(b1));
+}
+__device__ __forceinline__ void dldsm4(uint32_t addr, uint32_t (&r)[4]) {
+  asm volatile("ldmatrix.sync.aligned.m8n8.x4.shared.b16 {%0,%1,%2,%3}, [%4];"
+               : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]) : "r"(addr));
+}
+__device__ __forceinline__ void dldsm4t(uint32_t addr, uint32_t (&r)[4]) {
+  asm volatile("ldmatrix.sync.aligned.m8n8.x4.trans.shared.b16 {%0,%1,%2,%3}, [%4];"
+               : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]) : "r"(addr));
+}
+__device__ __forceinline__ void dldsm2(uint32_t addr, uint32_t &r0, uint32_t &r1) {
+  asm volatile("ldmatrix.sync.aligned.m8n8.x2.shared.b16 {%0,%1}, [%2];" : "=r"(r0), "=r"(r1) : "r"(addr));
+}
+__device__ __forceinline__ uint32_t dsm(const void *p) {
+  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+
+template <int D>
+struct PoolSmem {
+  static constexpr int ZS = D + 8;         // halves per Z row (16-byte rows, ldmatrix conflict-free)
+  static constexpr int WS = CH + 8;        // halves per W row
+  __half zh[CH * ZS], zl[CH * ZS];
+  __half mh[KHMAX * ZS], ml[KHMAX * ZS];   // Mᵀ [kh][c]
+  __half wh[KHMAX * WS], wl[KHMAX * WS];   // softmax weights [kh][row]
+  float sc[CH][KHMAX + 1];
+  float cst[KHMAX], mrun[KHMAX], lrun[KHMAX], scl[KHMAX];
+};
+
+template <int D>
+__global__ void __launch_bounds__(DT) set_decoder_pool_mma_kernel(const DecArgs a, const float *__restrict__ prep,
+                                                                  float *__restrict__ part) {
+  extern __shared__ __align__(16) unsigned char pool_raw[];
+  PoolSmem<D> &S = *reinterpret_cast<PoolSmem<D> *>(pool_raw);
+  constexpr int ZS = PoolSmem<D>::ZS, WS = PoolSmem<D>::WS;
+  constexpr int NTP = D >= 128 ? D / 128 : 1;   // n-tile pairs of P per warp (D = 128: 8 warps x 16 columns)
+  const int KH = a.k * a.heads;
+  const int t = threadIdx.x, warp = t >> 5, lane = t & 31, g = lane >> 2, tq = lane & 3;
+  const int gi = blockIdx.x, sp = blockIdx.y;
+  pdl_trigger();
+  pdl_wait();
+  const long g0 = a.node_off[gi], len = a.node_off[gi + 1] - g0;
+  const long u0 = g0 + len * sp / SPLIT, u1 = g0 + len * (sp + 1) / SPLIT;
+  // Mᵀ (columns kh >= KH zero) and the offsets
+  for (int i = t; i < KHMAX * D; i += DT) {
+    const int kh = i / D, c = i % D;
+    const float v = kh < KH ? __ldg(prep + c * KHMAX + kh) : 0.f;
+    const __half h = __float2half_rn(v);
+    S.mh[kh * ZS + c] = h;
+    S.ml[kh * ZS + c] = __float2half_rn(v - __half2float(h));
+  }
+  if (t < KHMAX) {
+    S.cst[t] = t < KH ? prep[D * KHMAX + t] : 0.f;
+    S.mrun[t] = -INFINITY;
+    S.lrun[t] = 0.f;
+  }
+  // P accumulators: warp owns n-tiles [warp·2·NTP/2 ...]: for D = 128, n-tiles 2w, 2w + 1
+  float pacc[2 * NTP][4];
+#pragma unroll
+  for (int n = 0; n < 2 * NTP; ++n) pacc[n][0] = pacc[n][1] = pacc[n][2] = pacc[n][3] = 0.f;
+  const int nbase = warp * 2 * NTP;        // first n-tile of this warp (8-column tiles)
+  const bool pw = nbase * 8 < D;           // warps beyond D/8/(2·NTP) idle in the P product
+  __syncthreads();
+  for (long n0 = u0; n0 < u1; n0 += CH) {
+    const int rows = int(min(long(CH), u1 - n0));
+    // ---- Z chunk -> fp16 hi / lo (rows past the range zero)
+    for (int i = t; i < CH * (D / 4); i += DT) {
+      const int r = i / (D / 4), c = (i % (D / 4)) * 4;
+      float4 z = make_float4(0.f, 0.f, 0.f, 0.f);
+      if (r < rows) z = __ldg(reinterpret_cast<const float4 *>(a.Z + (n0 + r) * D + c));
+      uint32_t h0, l0, h1, l1;
+      dsplit_h2(z.x, z.y, h0, l0);
+      dsplit_h2(z.z, z.w, h1, l1);
+      *reinterpret_cast<uint2 *>(&S.zh[r * ZS + c]) = make_uint2(h0, h1);
+      *reinterpret_cast<uint2 *>(&S.zl[r * ZS + c]) = make_uint2(l0, l1);
+    }
+    __syncthreads();
+    // ---- scores: warp w < 4 -> rows (w >> 1)·16.., seeds·heads (w & 1)·8..
+    if (warp < 4) {
+      const int mt = warp >> 1, nt = warp & 1;
+      float c4[4] = {0.f, 0.f, 0.f, 0.f};
+      const int arow = mt * 16 + (lane & 7) + ((lane >> 3) & 1) * 8, acol = (lane >> 4) * 8;
+      const int brow = nt * 8 + (lane & 7), bcol = ((lane >> 3) & 1) * 8;
+#pragma unroll
+      for (int ks = 0; ks < D / 16; ++ks) {
+        uint32_t ah[4], al[4], bh0, bh1, bl0, bl1;
+        dldsm4(dsm(&S.zh[arow * ZS + ks * 16 + acol]), ah);
+        dldsm4(dsm(&S.zl[arow * ZS + ks * 16 + acol]), al);
+        dldsm2(dsm(&S.mh[brow * ZS + ks * 16 + bcol]), bh0, bh1);
+        dldsm2(dsm(&S.ml[brow * ZS + ks * 16 + bcol]), bl0, bl1);
+        dmma(c4, al, bh0, bh1);
+        dmma(c4, ah, bl0, bl1);
+        dmma(c4, ah, bh0, bh1);
+      }
+      const int r0 = mt * 16 + g, col = nt * 8 + 2 * tq;
+      S.sc[r0][col] = r0 < rows ? c4[0] + S.cst[col] : -INFINITY;
+      S.sc[r0][col + 1] = r0 < rows ? c4[1] + S.cst[col + 1] : -INFINITY;
+      S.sc[r0 + 8][col] = r0 + 8 < rows ? c4[2] + S.cst[col] : -INFINITY;
+      S.sc[r0 + 8][col + 1] = r0 + 8 < rows ? c4[3] + S.cst[col + 1] : -INFINITY;
+    }
+    __syncthreads();
+    // ---- online softmax per (seed, head) column over the chunk's rows: warp per column
+    for (int kh = warp; kh < KHMAX; kh += NW) {
+      const float sv = S.sc[lane][kh];
+      float cm = sv;
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) cm = fmaxf(cm, __shfl_xor_sync(0xffffffffu, cm, o));
+      const float mold = S.mrun[kh];
+      const float mn = fmaxf(mold, cm);
+      const float ref = mn == -INFINITY ? 0.f : mn;
+      const float w = kh < KH ? ex2((sv - ref) * L2E) : 0.f;      // rows past the range: 0
+      float ws = w;
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) ws += __shfl_xor_sync(0xffffffffu, ws, o);
+      const __half wh = __float2half_rn(w);
+      S.wh[kh * WS + lane] = wh;
+      S.wl[kh * WS + lane] = __float2half_rn(w - __half2float(wh));
+      if (lane == 0) {
+        const float f = ex2((mold - ref) * L2E);                   // 0 on the first chunk
+        S.scl[kh] = f;
+        S.lrun[kh] = S.lrun[kh] * f + ws;
+        S.mrun[kh] = mn;
+      }
+    }
+    __syncthreads();
+    // ---- P[16][D] = P · scl + W[16][32] · Z[32][D]
+    if (pw) {
+      const float fa = S.scl[g], fb = S.scl[g + 8];
+#pragma unroll
+      for (int n = 0; n < 2 * NTP; ++n) {
+        pacc[n][0] *= fa; pacc[n][1] *= fa; pacc[n][2] *= fb; pacc[n][3] *= fb;
+      }
+      const int arow = (lane & 7) + ((lane >> 3) & 1) * 8, acol = (lane >> 4) * 8;
+#pragma unroll
+      for (int ks = 0; ks < CH / 16; ++ks) {
+        uint32_t ah[4], al[4];
+        dldsm4(dsm(&S.wh[arow * WS + ks * 16 + acol]), ah);
+        dldsm4(dsm(&S.wl[arow * WS + ks * 16 + acol]), al);
+        const int brow = ks * 16 + (lane & 7) + ((lane >> 3) & 1) * 8;
+#pragma unroll
+        for (int np = 0; np < NTP; ++np) {
+          const int bcol = (nbase + 2 * np + (lane >> 4)) * 8;
+          uint32_t bh[4], bl[4];
+          dldsm4t(dsm(&S.zh[brow * ZS + bcol]), bh);
+          dldsm4t(dsm(&S.zl[brow * ZS + bcol]), bl);
+          dmma(pacc[2 * np], al, bh[0], bh[1]);
+          dmma(pacc[2 * np], ah, bl[0], bl[1]);
+          dmma(pacc[2 * np], ah, bh[0], bh[1]);
+          dmma(pacc[2 * np + 1], al, bh[2], bh[3]);
+          dmma(pacc[2 * np + 1], ah, bl[2], bl[3]);
+          dmma(pacc[2 * np + 1], ah, bh[2], bh[3]);
+        }
+      }
+    }
+    __syncthreads();
+  }
+  float *out = part + (long(gi) * SPLIT + sp) * part_stride<D>();
+  if (pw) {
+#pragma unroll
+    for (int n = 0; n < 2 * NTP; ++n) {
+      const int c = (nbase + n) * 8 + 2 * tq;
+      if (g < KH) *reinterpret_cast<float2 *>(out + g * D + c) = make_float2(pacc[n][0], pacc[n][1]);
+      if (g + 8 < KH) *reinterpret_cast<float2 *>(out + (g + 8) * D + c) = make_float2(pacc[n][2], pacc[n][3]);
+    }
+  }
+  if (t < KH) {
+    out[KHMAX * D + t] = S.mrun[t];
+    out[KHMAX * D + KHMAX + t] = S.lrun[t];
+  }
+}
+
 // GPC graphs per CTA: combine each graph's SPLIT pool partials in fixed order, then the
 // MAB / SAB / FFN chain and the head as GEMVs over all GPC·k vectors of the CTA (every weight
 // row read from L2 once per CTA serves GPC graphs).
@@ -504,7 +692,12 @@ int launch_set_decoder(const occu_ctx *ctx, const DevCsr &csr, const float *hL, 
   const size_t smem_tail = (D == 64 ? tail_smem_floats<64>(cf.d_h) : tail_smem_floats<128>(cf.d_h)) * 4;
   const dim3 gpool(csr.B, SPLIT);
   int nprep = 0;
-  auto run = [&](auto prepk, auto poolk, auto tailk) {
+  static const bool simt_pool = [] {
+    const char *e = getenv("OCCU_DEC_POOL_SIMT");
+    return e && atoi(e) != 0;
+  }();
+  const size_t smem_mma = D == 64 ? sizeof(PoolSmem<64>) : sizeof(PoolSmem<128>);
+  auto run = [&](auto prepk, auto poolk, auto poolm, auto tailk) {
     if (ctx->dprep_version != ctx->params_version) {   // parameters changed: rebuild M, c
       OCCU_PROF_BEGIN(ctx, "set_decoder_prep", st);
       prepk<<<1, DT, 0, st>>>(a, prep);
@@ -513,8 +706,13 @@ int launch_set_decoder(const occu_ctx *ctx, const DevCsr &csr, const float *hL, 
       ++nprep;
     }
     OCCU_PROF_BEGIN(ctx, "set_decoder_pool", st);
-    cudaFuncSetAttribute(poolk, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem_pool));
-    launch_pdl(ctx->pdl & 8, poolk, gpool, DT, smem_pool, st, a, (const float *)prep, part);
+    if (simt_pool) {
+      cudaFuncSetAttribute(poolk, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem_pool));
+      launch_pdl(ctx->pdl & 8, poolk, gpool, DT, smem_pool, st, a, (const float *)prep, part);
+    } else {
+      cudaFuncSetAttribute(poolm, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem_mma));
+      launch_pdl(ctx->pdl & 8, poolm, gpool, DT, smem_mma, st, a, (const float *)prep, part);
+    }
     OCCU_PROF_END(ctx);
     OCCU_PROF_BEGIN(ctx, "set_decoder", st);
     cudaFuncSetAttribute(tailk, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem_tail));
@@ -522,9 +720,11 @@ int launch_set_decoder(const occu_ctx *ctx, const DevCsr &csr, const float *hL, 
     OCCU_PROF_END(ctx);
   };
   if (D == 64)
-    run(set_decoder_prep_kernel<64>, set_decoder_pool_kernel<64>, set_decoder_kernel<64>);
+    run(set_decoder_prep_kernel<64>, set_decoder_pool_kernel<64>, set_decoder_pool_mma_kernel<64>,
+        set_decoder_kernel<64>);
   else
-    run(set_decoder_prep_kernel<128>, set_decoder_pool_kernel<128>, set_decoder_kernel<128>);
+    run(set_decoder_prep_kernel<128>, set_decoder_pool_kernel<128>, set_decoder_pool_mma_kernel<128>,
+        set_decoder_kernel<128>);
   const cudaError_t e = cudaGetLastError();
   return e == cudaSuccess ? n + 2 + nprep : -int(e);
 }
