@@ -800,6 +800,19 @@ def main():
             del cg, m1g
         except Exception as ex:                       # noqa: BLE001 — reported, not hidden
             cfg1["cuda_graph"] = {"unavailable": str(ex)[:200]}
+        # the single-CTA small-batch kernel (opt-in, occu_set_small_batch_kernel)
+        m1.set_small_batch_kernel(True)
+        for _ in range(20):
+            f1()
+        torch.cuda.synchronize()
+        e0.record(stream)
+        for _ in range(reps):
+            f1()
+        e1.record(stream)
+        torch.cuda.synchronize()
+        uss = max_over_ranks(e0.elapsed_time(e1) * 1e3 / reps)
+        cfg1["single_cta_kernel"] = {"value": world * 1e6 / uss, "unit": "graphs/s", "us_per_graph": uss,
+                                     "launches_per_forward": m1.last_launch_count()}
         del m1
 
     # ---- CFG4 / CFG5 (BASELINE.json configs[3], configs[4]): the 20-family mixture.  Every

@@ -1,0 +1,261 @@
+// Small-batch forward (CFG1: "latency-bound ... Target: one persistent CTA"):
+// a whole batch of at most 64 nodes and 128 edges (e.g. one LeNet-5 training graph, 39 nodes
+// / 52 edges) runs the complete forward of §8(a) — a1 edge permutation, per layer a2 node
+// transform, a3 edge transform, a4 channel-softmax gate (reading A), a5/a6 gather and
+// segmented sum, then a7 readout and a8 head — inside ONE CTA with every activation in shared
+// memory: one launch instead of ~9, no HBM round trips between steps.  FP32 on CUDA cores
+// (a few hundred kFLOP per layer; tensor-core tiles of 128 rows would be mostly padding).
+// Fixed summation orders (deterministic); P141-P151, P125.
+#include <cuda_runtime.h>
+#include <math.h>
+#include <stdint.h>
+
+#include <algorithm>
+
+#include "occu_internal.h"
+
+namespace occu {
+namespace {
+
+constexpr int SNMAX = 64, SEMAX = 128, SKMAX = 128, ST = 1024;   // 32 warps: latency hiding on one SM
+constexpr size_t SMEM_MAX = 220 * 1024;
+
+struct SmallArgs {
+  const float *nf, *ef;                      // [N][F_n], [E][F_e] (input edge order)
+  const int32_t *node_off, *in_ptr, *in_src, *in_dst, *in_eid, *node_graph;
+  const float *P;                            // flat parameters
+  size_t W_u[8], W_e[8], W_m[8], a_s[8], a_d[8];
+  size_t W_1, b_1, w_2, b_2;
+  int L, F_n, F_e, d, d_h, B, N, E, mean, SK;     // SK = row stride of H / Ein (max width)
+  float slope;
+  float *r, *c, *yhat;                       // [B][d], [B][d_h], [B]
+};
+
+__device__ __forceinline__ float lrelu_s(float x, float s) { return x > 0.f ? x : s * x; }
+
+// Every global -> shared copy is a 4-byte cp.async (no register round trip, all in flight at
+// once); weights land with row stride K + 1 (the thread-per-output GEMM reads W[n][k] for 32
+// consecutive n: conflict-free).
+__device__ __forceinline__ void cpa4(void *dst, const void *src) {
+  asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(static_cast<uint32_t>(__cvta_generic_to_shared(dst))),
+               "l"(src) : "memory");
+}
+__device__ __forceinline__ void cpa_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void cpa_wait() { asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory"); }
+
+__device__ __forceinline__ void stage_w(const float *__restrict__ W, int Nout, int K, float *Ws) {
+  for (int i = threadIdx.x; i < Nout * K; i += ST) cpa4(Ws + (i / K) * (K + 1) + i % K, W + i);
+  cpa_commit();
+}
+
+// Y[r][n] = Σ_k X[r][k] Ws[n][k] over rows r < R, outputs n < Nout; thread per (r, n), four
+// independent partial sums, fixed order.
+__device__ __forceinline__ void small_gemm(const float *X, int ldx, int R, int K, const float *Ws,
+                                           int Nout, float *Y, int ldy) {
+  for (int i = threadIdx.x; i < R * Nout; i += ST) {
+    const int r = i / Nout, n = i % Nout;
+    const float *x = X + r * ldx;
+    const float *w = Ws + n * (K + 1);
+    float a0 = 0.f, a1 = 0.f, a2 = 0.f, a3 = 0.f;
+    int k = 0;
+    for (; k + 3 < K; k += 4) {
+      a0 = fmaf(x[k], w[k], a0);
+      a1 = fmaf(x[k + 1], w[k + 1], a1);
+      a2 = fmaf(x[k + 2], w[k + 2], a2);
+      a3 = fmaf(x[k + 3], w[k + 3], a3);
+    }
+    for (; k < K; ++k) a0 = fmaf(x[k], w[k], a0);
+    Y[r * ldy + n] = (a0 + a1) + (a2 + a3);
+  }
+}
+
+__global__ void __launch_bounds__(ST, 1) small_forward_kernel(const SmallArgs a) {
+  extern __shared__ float ssm[];
+  const int d = a.d, N = a.N, E = a.E, SK = a.SK;
+  float *H = ssm;                              // [N][SK] layer input h
+  float *Hb = H + N * SK;                      // [N][d]  h̄
+  float *pq = Hb + N * d;                      // [2][SNMAX]  p, q
+  float *E0 = pq + 2 * SNMAX;                  // [E][F_e] layer-1 edge input (in-CSR order)
+  float *Ev = E0 + E * a.F_e;                  // [E][d]  z / logits / gates
+  float *Ea = Ev + E * d;                      // [E][d]  e' (ping)
+  float *Eb = Ea + E * d;                      // [E][d]  e' (pong)
+  float *Wa = Eb + E * d;                      // [d][SK + 1] weight slot A (W_u, W_m)
+  float *Wb = Wa + d * (SK + 1);               // [d][SK + 1] weight slot B (W_e)
+  int32_t *cs = reinterpret_cast<int32_t *>(Wb + d * (SK + 1));
+  int32_t *iptr = cs, *isrc = cs + (N + 1), *idst = isrc + E, *ieid = idst + E;
+  const int t = threadIdx.x, warp = t >> 5, lane = t & 31;
+  pdl_trigger();
+  pdl_wait();
+  // a1: CSR, node features, first layer's weights; then the in-CSR-ordered edge features
+  for (int i = t; i <= N; i += ST) cpa4(iptr + i, a.in_ptr + i);
+  for (int i = t; i < E; i += ST) {
+    cpa4(isrc + i, a.in_src + i);
+    cpa4(idst + i, a.in_dst + i);
+    cpa4(ieid + i, a.in_eid + i);
+  }
+  for (int i = t; i < N * a.F_n; i += ST) cpa4(H + (i / a.F_n) * SK + i % a.F_n, a.nf + i);
+  cpa_commit();
+  stage_w(a.P + a.W_u[0], d, a.F_n, Wa);
+  stage_w(a.P + a.W_e[0], d, a.F_e, Wb);
+  cpa_wait<2>();                               // CSR + node features
+  __syncthreads();
+  for (int i = t; i < E * a.F_e; i += ST) {
+    const int k = i / a.F_e, c = i % a.F_e;
+    cpa4(E0 + i, a.ef + size_t(ieid[k]) * a.F_e + c);
+  }
+  cpa_commit();                                // groups in flight: W_u, W_e, E0
+  int K = a.F_n, Ke = a.F_e;
+  const float *Ein = E0;
+  int lde = a.F_e;
+  float *Eout = Ea;
+  for (int l = 0; l < a.L; ++l) {
+    const float *P = a.P;
+    // a2: h̄ = LReLU(h W_uᵀ); p = h̄·a_s, q = h̄·a_d          (groups: W_u, W_e[, E0])
+    if (l == 0) cpa_wait<2>(); else cpa_wait<1>();
+    __syncthreads();
+    small_gemm(H, SK, N, K, Wa, d, Hb, d);
+    __syncthreads();
+    stage_w(P + a.W_m[l], d, d, Wa);           // slot A: W_m (W_u consumed)
+    for (int i = t; i < N * d; i += ST) Hb[i] = lrelu_s(Hb[i], a.slope);
+    __syncthreads();
+    for (int u = warp; u < N; u += ST / 32) {
+      float ps = 0.f, qs = 0.f;
+      for (int c = lane; c < d; c += 32) {
+        ps = fmaf(Hb[u * d + c], __ldg(P + a.a_s[l] + c), ps);
+        qs = fmaf(Hb[u * d + c], __ldg(P + a.a_d[l] + c), qs);
+      }
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) {
+        ps += __shfl_xor_sync(0xffffffffu, ps, o);
+        qs += __shfl_xor_sync(0xffffffffu, qs, o);
+      }
+      if (lane == 0) {
+        pq[u] = ps;
+        pq[SNMAX + u] = qs;
+      }
+    }
+    // a3: z = e_in W_eᵀ, e' = σ(α z), α = p[src] + q[dst]     (groups: W_e[, E0], W_m)
+    cpa_wait<1>();
+    __syncthreads();
+    small_gemm(Ein, lde, E, Ke, Wb, d, Ev, d);
+    __syncthreads();
+    if (l + 1 < a.L) stage_w(P + a.W_e[l + 1], d, d, Wb);      // slot B: next W_e
+    for (int i = t; i < E * d; i += ST) {
+      const int k = i / d;
+      const float al = pq[isrc[k]] + pq[SNMAX + idst[k]];
+      Eout[i] = 1.f / (1.f + expf(-al * Ev[i]));
+    }
+    // a4: logits W_m e', softmax over the d channels (warp per edge)
+    if (l + 1 < a.L) cpa_wait<1>(); else cpa_wait<0>();
+    __syncthreads();
+    small_gemm(Eout, d, E, d, Wa, d, Ev, d);
+    __syncthreads();
+    if (l + 1 < a.L) stage_w(P + a.W_u[l + 1], d, d, Wa);      // slot A: next W_u
+    for (int k = warp; k < E; k += ST / 32) {
+      float m = -INFINITY;
+      for (int c = lane; c < d; c += 32) m = fmaxf(m, Ev[k * d + c]);
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, o));
+      float s = 0.f;
+      for (int c = lane; c < d; c += 32) {
+        const float x = expf(Ev[k * d + c] - m);
+        Ev[k * d + c] = x;
+        s += x;
+      }
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+      const float inv = 1.f / s;
+      for (int c = lane; c < d; c += 32) Ev[k * d + c] *= inv;
+    }
+    __syncthreads();
+    // a5/a6: h[t] = LReLU(Σ_{k∈seg(t)} g_k ⊙ h̄[s_k]) (÷ deg for MEAN), ascending k
+    for (int i = t; i < N * d; i += ST) {
+      const int v = i / d, c = i % d;
+      const int k0 = iptr[v], k1 = iptr[v + 1];
+      float acc = 0.f;
+      for (int k = k0; k < k1; ++k) acc = fmaf(Ev[k * d + c], Hb[isrc[k] * d + c], acc);
+      if (a.mean) acc /= float(k1 > k0 ? k1 - k0 : 1);
+      H[v * SK + c] = lrelu_s(acc, a.slope);
+    }
+    __syncthreads();
+    Ein = Eout;                                // e' feeds the next layer (ping-pong)
+    lde = d;
+    Eout = Eout == Ea ? Eb : Ea;
+    K = d;
+    Ke = d;
+  }
+  // a7: per-graph mean readout; a8: head (warp per graph for the final dot)
+  for (int i = t; i < a.B * d; i += ST) {
+    const int b = i / d, c = i % d;
+    const int u0 = __ldg(a.node_off + b), u1 = __ldg(a.node_off + b + 1);
+    float s = 0.f;
+    for (int u = u0; u < u1; ++u) s += H[u * SK + c];
+    a.r[i] = s / float(u1 - u0);
+  }
+  __syncthreads();
+  for (int i = t; i < a.B * a.d_h; i += ST) {
+    const int b = i / a.d_h, n = i % a.d_h;
+    float s0 = __ldg(a.P + a.b_1 + n), s1 = 0.f, s2 = 0.f, s3 = 0.f;
+    const float *w = a.P + a.W_1 + size_t(n) * d, *rr = a.r + b * d;
+    for (int c = 0; c < d; c += 4) {
+      s0 = fmaf(__ldg(w + c), rr[c], s0);
+      s1 = fmaf(__ldg(w + c + 1), rr[c + 1], s1);
+      s2 = fmaf(__ldg(w + c + 2), rr[c + 2], s2);
+      s3 = fmaf(__ldg(w + c + 3), rr[c + 3], s3);
+    }
+    a.c[i] = (s0 + s1) + (s2 + s3);
+  }
+  __syncthreads();
+  for (int b = warp; b < a.B; b += ST / 32) {
+    float s = 0.f;
+    for (int n = lane; n < a.d_h; n += 32) s = fmaf(__ldg(a.P + a.w_2 + n), lrelu_s(a.c[b * a.d_h + n], a.slope), s);
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+    if (lane == 0) a.yhat[b] = s + __ldg(a.P + a.b_2);
+  }
+}
+
+}  // namespace
+
+static size_t small_smem(const occu_config &c, const DevCsr &csr) {
+  const int sk = std::max(c.F_n, std::max(c.F_e, c.d));
+  return size_t(csr.N * sk + csr.N * c.d + 2 * SNMAX + csr.E * c.F_e + 3 * csr.E * c.d +
+                2 * c.d * (sk + 1) + (csr.N + 1) + 3 * csr.E) * 4;
+}
+
+bool small_forward_ok(const occu_ctx *ctx, const DevCsr &csr) {
+  const occu_config &c = ctx->cfg;
+  return c.prec == OCCU_FP32 && c.msg == OCCU_MSG_CHANNEL_SOFTMAX && c.readout == OCCU_READOUT_MEAN &&
+         c.graphormer == 0 && c.L <= 8 && csr.N >= 1 && csr.N <= SNMAX && csr.E <= SEMAX &&
+         c.F_n <= SKMAX && c.F_e <= SKMAX && c.d <= SKMAX && small_smem(c, csr) <= SMEM_MAX;
+}
+
+int launch_small_forward(const occu_ctx *ctx, const DevCsr &csr, const float *nf, const float *ef,
+                         float *r, float *cvec, float *yhat, cudaStream_t st) {
+  const occu_config &c = ctx->cfg;
+  const ParamLayout &L = ctx->layout;
+  SmallArgs a{};
+  a.nf = nf; a.ef = ef;
+  a.node_off = csr.node_off; a.in_ptr = csr.in_ptr; a.in_src = csr.in_src; a.in_dst = csr.in_dst;
+  a.in_eid = csr.in_eid; a.node_graph = csr.node_graph;
+  a.P = ctx->params.as<float>();
+  for (int i = 0; i < c.L; ++i) {
+    a.W_u[i] = L.W_u[i]; a.W_e[i] = L.W_e[i]; a.W_m[i] = L.W_m[i]; a.a_s[i] = L.a_s[i]; a.a_d[i] = L.a_d[i];
+  }
+  a.W_1 = L.W_1; a.b_1 = L.b_1; a.w_2 = L.w_2; a.b_2 = L.b_2;
+  a.L = c.L; a.F_n = c.F_n; a.F_e = c.F_e; a.d = c.d; a.d_h = c.d_h;
+  a.B = csr.B; a.N = csr.N; a.E = csr.E; a.mean = c.aggr == OCCU_AGGR_MEAN;
+  a.slope = c.slope;
+  a.SK = std::max(c.F_n, std::max(c.F_e, c.d));   // H row stride; W staged with K + 1
+  a.r = r; a.c = cvec; a.yhat = yhat;
+  const size_t smem = small_smem(c, csr);
+  cudaFuncSetAttribute(small_forward_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
+  OCCU_PROF_BEGIN(ctx, "small_forward", st);
+  small_forward_kernel<<<1, ST, smem, st>>>(a);
+  OCCU_PROF_END(ctx);
+  const cudaError_t e = cudaGetLastError();
+  return e == cudaSuccess ? 1 : -int(e);
+}
+
+}  // namespace occu

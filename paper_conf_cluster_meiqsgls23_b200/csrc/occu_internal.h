@@ -126,6 +126,8 @@ struct occu_ctx {
   occu::DevCsr last_csr;   // geometry of the last forward (for occu_get_tensor)
   bool have_forward = false;
   bool h_last_stored = true;   // false: the last forward kept only readout partials of h_L
+  bool small_fwd = false;      // the last forward ran the single-CTA small-batch kernel
+  bool small_enabled = false;  // occu_set_small_batch_kernel: single-CTA forward for tiny batches
   int64_t launches = 0;
   mutable occu::Profiler prof;
   // occu_predict_async: H2D on a copy stream into staging slot a_slot, compute on `stream`
@@ -237,6 +239,9 @@ int launch_readout_head(const occu_ctx *ctx, const DevCsr &csr, const float *h, 
 // NEXT-2 readout (kernels_decoder.cu): Z = FFN(h_L) on tensor cores (T = ReLU(h W1ᵀ + b1),
 // Z = T W2ᵀ + b2), then per graph the k-seed attention pool over Z, the MAB / SAB / FFN tail
 // and the head; r receives the flattened decoder output [B][k·d].
+bool small_forward_ok(const occu_ctx *ctx, const DevCsr &csr);
+int launch_small_forward(const occu_ctx *ctx, const DevCsr &csr, const float *nf, const float *ef,
+                         float *r, float *cvec, float *yhat, cudaStream_t st);
 int launch_graphormer_layer(const occu_ctx *ctx, const DevCsr &csr, int j, const float *h_in,
                             float *h_out, float *X, float *QKV, float *O, cudaStream_t st);
 int launch_bias_add_tc(const occu_ctx *ctx, const float *A, int K, int R, int wkind, int layer,

@@ -257,6 +257,17 @@ occu_status forward(occu_ctx *ctx, const DevCsr &csr, const float *nf, const flo
   const float *P = ctx->params.as<float>();
   const bool bf = c.prec == OCCU_BF16;        // kernel path 0 only (occu_set_kernel_path)
   const bool tc = bf || (ctx->path != 1 && tc_supported(c));
+  if (!save_all && ctx->path == 0 && ctx->small_enabled && small_forward_ok(ctx, csr)) {
+    // CFG1-sized batches: the whole forward in one CTA (kernels_small.cu)
+    LK(launch_small_forward(ctx, csr, nf, ef, w.r.as<float>(), w.c.as<float>(), w.yhat.as<float>(), s),
+       "small forward");
+    ctx->small_fwd = true;
+    ctx->h_last_stored = false;
+    ctx->last_csr = csr;
+    ctx->have_forward = true;
+    return OCCU_OK;
+  }
+  ctx->small_fwd = false;
   // Tensor-core path fusions: a1's edge permutation folded into the layer-1 edge kernel,
   // and the readout's node sums folded into the last aggregation (chunk partials).
   const bool fuse_e0 = tc && c.F_e <= 16;
@@ -820,6 +831,12 @@ occu_status occu_load_state(occu_ctx *ctx, const char *path) {
   return OCCU_OK;
 }
 
+occu_status occu_set_small_batch_kernel(occu_ctx *ctx, int enable) {
+  if (!ctx) return fail(nullptr, OCCU_EINVAL, "ctx is NULL");
+  ctx->small_enabled = enable != 0;
+  return OCCU_OK;
+}
+
 occu_status occu_set_kernel_path(occu_ctx *ctx, int path) {
   if (!ctx) return fail(nullptr, OCCU_EINVAL, "ctx is NULL");
   if (path < 0 || path > 2)
@@ -849,6 +866,8 @@ occu_status occu_get_tensor(occu_ctx *ctx, int32_t which, int32_t layer, void *h
   const int d = ctx->cfg.d;
   const bool per_layer = which <= OCCU_T_H;
   if (per_layer && (layer < 0 || layer >= ctx->cfg.L)) return fail(ctx, OCCU_EINVAL, "bad layer");
+  if (per_layer && ctx->small_fwd)
+    return fail(ctx, OCCU_ENOTREADY, "the last forward ran the single-CTA small-batch kernel (no per-layer tensors; set keep_intermediates)");
   if (which == OCCU_T_GPH && (layer < 0 || layer >= ctx->cfg.graphormer))
     return fail(ctx, OCCU_EINVAL, "bad Graphormer layer");
   const void *src = nullptr;

@@ -32,7 +32,7 @@ EXPORTS = [
     "occu_dist_init", "occu_save_state", "occu_load_state", "occu_set_keep_intermediates",
     "occu_get_tensor", "occu_last_launch_count", "occu_last_error", "occu_set_profiling",
     "occu_profile_reset", "occu_profile_query", "occu_set_kernel_path", "occu_pack_jobs",
-    "occu_template_create", "occu_template_destroy", "occu_synthesize",
+    "occu_template_create", "occu_template_destroy", "occu_synthesize", "occu_set_small_batch_kernel",
 ]
 
 
@@ -115,6 +115,7 @@ def lib():
             "occu_last_error": ([VP], C.c_char_p),
             "occu_set_profiling": ([VP, C.c_int], I32),
             "occu_set_kernel_path": ([VP, C.c_int], I32),
+            "occu_set_small_batch_kernel": ([VP, C.c_int], I32),
             "occu_profile_reset": ([VP], I32),
             "occu_profile_query": ([VP, I32, P(C.c_char_p), P(C.c_double), P(C.c_int64)], I32),
         }
@@ -377,6 +378,9 @@ class Model:
         _check(lib().occu_load_state(self._ctx, path.encode()), self._ctx)
 
     # batches
+    def set_small_batch_kernel(self, enable: bool):
+        _check(lib().occu_set_small_batch_kernel(self._ctx, int(bool(enable))), self._ctx)
+
     # NEXT-4: on-device feature synthesis
     def template(self, t):
         """Upload one family template (occu_gen.templates.Template) to this ctx's device."""
