@@ -800,6 +800,20 @@ def main():
             del cg, m1g
         except Exception as ex:                       # noqa: BLE001 — reported, not hidden
             cfg1["cuda_graph"] = {"unavailable": str(ex)[:200]}
+        # the CUDA-core (SIMT) kernel path on the same graph
+        m1.set_kernel_path(1)
+        for _ in range(20):
+            f1()
+        torch.cuda.synchronize()
+        e0.record(stream)
+        for _ in range(reps):
+            f1()
+        e1.record(stream)
+        torch.cuda.synchronize()
+        usp = max_over_ranks(e0.elapsed_time(e1) * 1e3 / reps)
+        cfg1["simt_path"] = {"value": world * 1e6 / usp, "unit": "graphs/s", "us_per_graph": usp,
+                             "launches_per_forward": m1.last_launch_count()}
+        m1.set_kernel_path(0)
         # the single-CTA small-batch kernel (opt-in, occu_set_small_batch_kernel)
         m1.set_small_batch_kernel(True)
         for _ in range(20):
