@@ -179,3 +179,11 @@ def test_graphormer_parity_is_sensitive_to_the_attention():
     ref = oracle.forward(params, ocfg(c), oracle.pack(b.graphs), b.node_feat, b.edge_feat)
     got = m.get_tensor(occu.T_GPH, 0, (b.num_nodes, c.d))
     assert rel(got, ref["gph"][0]) > 5 * TOL
+
+
+def test_graphormer_cfg3_sized_graphs():
+    """Two BERT-base training graphs (~3k nodes each, CFG3's per-graph size): 47 key blocks
+    per query tile, every tile inside one graph; layer outputs and ŷ vs the float64 oracle."""
+    c = mk(3, 128, 1, 4)
+    b = configs.cfg3(512).subset([0, 300])
+    check(c, b, params_for(c, 31))
