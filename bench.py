@@ -333,6 +333,16 @@ def main():
             pg.barrier()
         torch.cuda.synchronize()
 
+    def work_imbalance(w):
+        """max / mean over ranks of this rank's work (nodes + edges); 1.0 = balanced."""
+        if not pg:
+            return 1.0
+        t_ = torch.tensor([float(w), float(w)], dtype=torch.float64, device=dev)
+        mx = t_[:1].clone()
+        pg.all_reduce(mx, op=pg.ReduceOp.MAX)
+        pg.all_reduce(t_[1:], op=pg.ReduceOp.SUM)
+        return float(mx.item() / (t_[1].item() / world))
+
     def max_over_ranks(v):
         if not pg:
             return v
@@ -875,7 +885,8 @@ def main():
                         "edges_per_microbatch": [bb.num_edges for bb in mb4],
                         "includes": "forward with saves, MSE, backward, "
                                     + ("NCCL allreduce, " if world > 1 else "") + "Adam",
-                        "sharding": "contiguous per-rank shards of the seeded mixture"}
+                        "sharding": "contiguous per-rank shards of the seeded mixture",
+                        "rank_work_imbalance": work_imbalance(sum(bb.num_nodes + bb.num_edges for bb in mb4))}
             c_, n_, e_, y_ = dev4[0]
             ent["loss_after"] = m4.train_step(c_, n_, e_, y_, 1e-3, global_num_graphs=gB4)
             cfg4[key] = ent
