@@ -62,7 +62,8 @@ typedef enum { OCCU_READOUT_MEAN = 0, OCCU_READOUT_SET_DECODER = 1 } occu_readou
 /* Model configuration.  L ANEE rounds of width d (64 or 128 in this build); raw feature
  * widths F_n (node, Table I) and F_e (edge); head hidden width d_h; LeakyReLU slope (R7,
  * 0.01); F_n, F_e multiples of 4.  msg = OCCU_MSG_NEIGHBOR_SOFTMAX (reading B, NEXT-1):
- * OCCU_FP32, kernel path 0.  readout: OCCU_READOUT_MEAN (a7, the north_star's segmented
+ * kernel path 0; OCCU_FP32 forward + training, OCCU_BF16 forward (training with OCCU_BF16
+ * returns OCCU_EINVAL: DESIGN.md R40).  readout: OCCU_READOUT_MEAN (a7, the north_star's segmented
  * mean; default when the trailing fields are zero) or OCCU_READOUT_SET_DECODER (P159-P205,
  * NEXT-2: Decoder(H) = FFN(SAB(PMA_k(H))) per graph, k seeds, `heads` attention heads, the
  * head reading the flattened k·d output; OCCU_FP32, kernel path 0, inference only: training
