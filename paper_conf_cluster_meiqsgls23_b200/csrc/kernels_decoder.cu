@@ -467,6 +467,7 @@ __global__ void __launch_bounds__(DT) set_decoder_pool_mma_kernel(const DecArgs 
       const __half wh = __float2half_rn(w);
       S.wh[kh * WS + lane] = wh;
       S.wl[kh * WS + lane] = __float2half_rn(w - __half2float(wh));
+      __syncwarp();                          // every lane has read mrun[kh] / lrun[kh]
       if (lane == 0) {
         const float f = ex2((mold - ref) * L2E);                   // 0 on the first chunk
         S.scl[kh] = f;

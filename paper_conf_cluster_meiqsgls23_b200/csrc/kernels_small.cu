@@ -112,7 +112,9 @@ __global__ void __launch_bounds__(ST, 1) small_forward_kernel(const SmallArgs a)
   for (int l = 0; l < a.L; ++l) {
     const float *P = a.P;
     // a2: h̄ = LReLU(h W_uᵀ); p = h̄·a_s, q = h̄·a_d          (groups: W_u, W_e[, E0])
-    if (l == 0) cpa_wait<2>(); else cpa_wait<1>();
+    // layer 0: W_u0 is the second of four groups (CSR + H, W_u0, W_e0, E0); later layers:
+    // W_u(l) is the most recent group (issued after W_e(l)), so everything must land
+    if (l == 0) cpa_wait<2>(); else cpa_wait<0>();
     __syncthreads();
     small_gemm(H, SK, N, K, Wa, d, Hb, d);
     __syncthreads();
