@@ -562,6 +562,28 @@ def main():
                               "+ FFN) -> mean readout -> head (P153-P157)"}
         del mg
 
+    # ---- the paper's model stack (P273: ANEE -> 2 Graphormer layers -> Set-Transformer decoder
+    # -> head; here L = 3 ANEE rounds at d = 128), FP32 and OCCU_BF16 (R41), same batch
+    paper_stack = None
+    if not args.no_bf16 and args.path == 0:
+        paper_stack = {"what": "ANEE x3 -> Graphormer x2 (4 heads) -> Set-Transformer decoder (k = 4, "
+                               "4 heads) -> head, CFG2 batch"}
+        for prec, key in ((occu.FP32, "f32"), (occu.BF16, "bf16")):
+            mps = occu.Model(occu.config(L=3, F_n=80, F_e=4, d=128, prec=prec, graphormer=2, heads=4,
+                                         readout=occu.READOUT_SET_DECODER, k=4),
+                             device=local, stream=stream.cuda_stream)
+            mps.init_weights(42)
+            outp = torch.empty_like(out)
+            fps = lambda: mps.predict(csr, nf, ef, outp)
+            timed(fps, args.warmup, mdl=mps)
+            bar()
+            tps, lps = timed(fps, args.steps, mdl=mps)
+            bar()
+            msps = max_over_ranks(float(np.sum(tps)) / args.steps)
+            paper_stack[key] = {"value": B * world / (msps * 1e-3), "unit": "graphs/s",
+                                "ms_per_step": msps, "dtype": key, "gpu_launches": lps}
+            del mps
+
     # ---- e2e through the public API with host buffers (pinned), pack included
     pin_nf = torch.from_numpy(batch.node_feat).pin_memory()
     pin_ef = torch.from_numpy(batch.edge_feat).pin_memory()
@@ -1069,6 +1091,7 @@ def main():
             "readingb": readingb,
             "decoder": decoder,
             "graphormer": graphormer,
+            "paper_stack": paper_stack,
             "train": train,
             "train_cfg3": train_cfg3,
             "cfg1": cfg1,

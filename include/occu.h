@@ -66,13 +66,14 @@ typedef enum { OCCU_READOUT_MEAN = 0, OCCU_READOUT_SET_DECODER = 1 } occu_readou
  * returns OCCU_EINVAL: DESIGN.md R40).  readout: OCCU_READOUT_MEAN (a7, the north_star's segmented
  * mean; default when the trailing fields are zero) or OCCU_READOUT_SET_DECODER (P159-P205,
  * NEXT-2: Decoder(H) = FFN(SAB(PMA_k(H))) per graph, k seeds, `heads` attention heads, the
- * head reading the flattened k·d output; OCCU_FP32, kernel path 0, inference only: training
- * returns OCCU_EINVAL); k in [1, 8], heads in {1, 2, 4, 8}, k·heads <= 16.
+ * head reading the flattened k·d output; kernel path 0, inference only: training returns
+ * OCCU_EINVAL; with OCCU_BF16 the decoder runs in FP32 on the BF16-stored h_L, R41);
+ * k in [1, 8], heads in {1, 2, 4, 8}, k·heads <= 16.
  * graphormer: number of Graphormer layers (P153-P157, NEXT-3; R35-R37) between the
  * last ANEE round and the readout, h̄ = MHA(LN(h)) + h, h' = FFN(LN(h̄)) + h̄ with
  * self-attention over each graph's own node set, `heads` heads (d / heads in {16, 32, 64});
- * 0 = none (default).  OCCU_FP32, kernel path 0, inference only (training returns
- * OCCU_EINVAL); graphormer in [0, 4]. */
+ * 0 = none (default).  Kernel path 0, inference only (training returns OCCU_EINVAL); with
+ * OCCU_BF16 the layers run in FP32 on the BF16-stored h_L (R41); graphormer in [0, 4]. */
 typedef struct {
   int32_t L, F_n, F_e, d, d_h;
   int32_t aggr;      /* occu_aggr */

@@ -309,6 +309,11 @@ def forward_bf16(params, cfg, pk, node_feat, edge_feat, rnd=None):
         layers.append(dict(P=P, hbar=hbar, p=p, q=q, alpha=alpha, z=z, e=e_new, g=g, A=A,
                            h=r16(h_f), h_f32=h_f))
         h, e = r16(h_f), e_new
+    if cfg.get("readout", 0) == 1 or cfg.get("graphormer", 0) > 0:
+        # R41: Graphormer layers / the decoder run in FP32 on the BF16-stored last h
+        f = dict(layers=layers, h0=np.asarray(node_feat, np.float64),
+                 e0=np.asarray(edge_feat, np.float64)[pk["in_eid"].astype(np.int64)])
+        return readout_stack(params, cfg, pk, f, layers[-1]["h"])
     n_b = np.diff(pk["node_off"].astype(np.int64))
     r = segment_sum(layers[-1]["h_f32"], pk["node_graph"].astype(np.int64), pk["num_graphs"]) / n_b[:, None]
     c = r @ params["W_1"].T + params["b_1"]                       # P125 (R12)
@@ -377,19 +382,14 @@ def graphormer_layer(H, params, j, heads):
     return ffn(Y, params, g + "F_") + Hb
 
 
-def forward(params, cfg, pk, node_feat, edge_feat):
-    """forward_anee, then cfg["graphormer"] Graphormer layers per graph (NEXT-3), then the
-    readout: the segmented mean (a7) or, with cfg["readout"] == 1, the Set-Transformer decoder
-    per graph (NEXT-2); then the MLP head on the (flattened) readout."""
-    f = forward_anee(params, cfg, pk, node_feat, edge_feat)
-    G = cfg.get("graphormer", 0)
-    if cfg.get("readout", 0) != 1 and G == 0:
-        return f
-    hL = f["layers"][-1]["h"]
+def readout_stack(params, cfg, pk, f, hL):
+    """cfg["graphormer"] Graphormer layers per graph (NEXT-3) on the last ANEE states hL, then
+    the readout — the segmented mean (a7) or, with cfg["readout"] == 1, the Set-Transformer
+    decoder per graph (NEXT-2) — and the MLP head on the (flattened) readout; fills f."""
     off = pk["node_off"].astype(np.int64)
     B = pk["num_graphs"]
     gph = []
-    for j in range(G):
+    for j in range(cfg.get("graphormer", 0)):
         hL = np.concatenate([graphormer_layer(hL[off[b]:off[b + 1]], params, j, cfg["heads"])
                              for b in range(B)])
         gph.append(hL)
@@ -404,6 +404,14 @@ def forward(params, cfg, pk, node_feat, edge_feat):
     o = leaky_relu(c, cfg["slope"])
     f.update(r=r, c=c, o=o, yhat=o @ params["w_2"] + params["b_2"][0])
     return f
+
+
+def forward(params, cfg, pk, node_feat, edge_feat):
+    """forward_anee, then (with Graphormer layers or the decoder readout) readout_stack."""
+    f = forward_anee(params, cfg, pk, node_feat, edge_feat)
+    if cfg.get("readout", 0) != 1 and cfg.get("graphormer", 0) == 0:
+        return f
+    return readout_stack(params, cfg, pk, f, f["layers"][-1]["h"])
 
 
 def predict(params, cfg, graphs, node_feat, edge_feat):

@@ -652,4 +652,30 @@ int launch_forward_layer_bf16(const occu_ctx *ctx, const DevCsr &csr, int layer,
   }
 }
 
+namespace {
+// exact BF16 -> FP32 widening, 8 elements per thread (16-byte loads)
+__global__ void __launch_bounds__(256) bf16_to_f32_kernel(const uint4 *__restrict__ src, size_t n8,
+                                                          float4 *__restrict__ dst) {
+  for (size_t i = blockIdx.x * size_t(256) + threadIdx.x; i < n8; i += size_t(gridDim.x) * 256) {
+    const uint4 v = __ldg(src + i);
+    dst[2 * i] = make_float4(__uint_as_float(v.x << 16), __uint_as_float(v.x & 0xFFFF0000u),
+                             __uint_as_float(v.y << 16), __uint_as_float(v.y & 0xFFFF0000u));
+    dst[2 * i + 1] = make_float4(__uint_as_float(v.z << 16), __uint_as_float(v.z & 0xFFFF0000u),
+                                 __uint_as_float(v.w << 16), __uint_as_float(v.w & 0xFFFF0000u));
+  }
+}
+}  // namespace
+
+int launch_bf16_to_f32(const occu_ctx *ctx, const void *src, size_t n, float *dst, cudaStream_t st) {
+  if (n % 8) return -int(cudaErrorInvalidValue);          // n = N·d, d in {64, 128}
+  const size_t n8 = n / 8;
+  const int grid = int(std::min<size_t>((n8 + 255) / 256, size_t(8) * ctx->num_sms));
+  if (n8 == 0) return 0;
+  OCCU_PROF_BEGIN(ctx, "bf16_to_f32", st);
+  bf16_to_f32_kernel<<<grid, 256, 0, st>>>(static_cast<const uint4 *>(src), n8, reinterpret_cast<float4 *>(dst));
+  OCCU_PROF_END(ctx);
+  const cudaError_t e = cudaGetLastError();
+  return e == cudaSuccess ? 1 : -int(e);
+}
+
 }  // namespace occu

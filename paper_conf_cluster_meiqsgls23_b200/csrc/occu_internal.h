@@ -69,6 +69,7 @@ struct Workspace {
   DevBuf dpool;            // decoder readout: pool partials [B][8][16·d + 32]
   std::vector<DevBuf> gh;  // Graphormer layer outputs [N][d] (per layer)
   DevBuf scsr, snf, sef, sdesc;   // occu_synthesize: batch CSR, node / edge rows, descriptors
+  DevBuf hf;               // OCCU_BF16 with Graphormer / decoder: h_L widened to FP32 (R41)
   DevBuf gx, gqkv, go;     // Graphormer scratch: LN output [N][d], Q|K|V [3][N][d], attention [N][d]
   void release_all();
 };
@@ -239,6 +240,7 @@ int launch_readout_head(const occu_ctx *ctx, const DevCsr &csr, const float *h, 
 // NEXT-2 readout (kernels_decoder.cu): Z = FFN(h_L) on tensor cores (T = ReLU(h W1ᵀ + b1),
 // Z = T W2ᵀ + b2), then per graph the k-seed attention pool over Z, the MAB / SAB / FFN tail
 // and the head; r receives the flattened decoder output [B][k·d].
+int launch_bf16_to_f32(const occu_ctx *ctx, const void *src, size_t n, float *dst, cudaStream_t st);
 bool small_forward_ok(const occu_ctx *ctx, const DevCsr &csr);
 int launch_small_forward(const occu_ctx *ctx, const DevCsr &csr, const float *nf, const float *ef,
                          float *r, float *cvec, float *yhat, cudaStream_t st);

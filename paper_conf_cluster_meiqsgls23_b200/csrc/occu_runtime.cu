@@ -48,7 +48,7 @@ void Workspace::release_all() {
                     &dy, &dc, &dr, &dh, &dhprev, &dP, &MG, &DV, &DZ, &deA, &deB, &dalpha,
                     &dpq, &partial, &loss, &tcpart, &dpart, &rpart, &anf[0], &anf[1],
                     &aef[0], &aef[1], &acsr[0], &acsr[1], &dT, &dZ, &dprep, &dpool, &gx, &gqkv, &go,
-                    &scsr, &snf, &sef, &sdesc};
+                    &scsr, &snf, &sef, &sdesc, &hf};
   for (DevBuf *b : bufs) b->release();
   for (auto *v : {&hbar, &p, &q, &e, &h, &gs, &gh})
     for (DevBuf &b : *v) b.release();
@@ -167,8 +167,8 @@ occu_status validate_cfg(const occu_config *c) {
   if (c->readout != OCCU_READOUT_MEAN && c->readout != OCCU_READOUT_SET_DECODER)
     return fail(nullptr, OCCU_EINVAL, "readout must be MEAN or SET_DECODER");
   if (c->readout == OCCU_READOUT_SET_DECODER) {
-    if (c->prec != OCCU_FP32 || c->F_n > 128)
-      return fail(nullptr, OCCU_EINVAL, "the Set-Transformer decoder readout runs in OCCU_FP32 on the tensor-core path");
+    if (c->F_n > 128)
+      return fail(nullptr, OCCU_EINVAL, "the Set-Transformer decoder readout runs on the tensor-core path (F_n <= 128)");
     if (c->k < 1 || c->k > 8 || !(c->heads == 1 || c->heads == 2 || c->heads == 4 || c->heads == 8) ||
         c->k * c->heads > 16 || c->d % c->heads)
       return fail(nullptr, OCCU_EINVAL, "decoder: k in [1,8], heads in {1,2,4,8}, k*heads <= 16");
@@ -176,8 +176,8 @@ occu_status validate_cfg(const occu_config *c) {
   if (c->graphormer < 0 || c->graphormer > 4)
     return fail(nullptr, OCCU_EINVAL, "graphormer must be in [0, 4]");
   if (c->graphormer > 0) {
-    if (c->prec != OCCU_FP32 || c->F_n > 128)
-      return fail(nullptr, OCCU_EINVAL, "Graphormer layers run in OCCU_FP32 on the tensor-core path");
+    if (c->F_n > 128)
+      return fail(nullptr, OCCU_EINVAL, "Graphormer layers run on the tensor-core path (F_n <= 128)");
     if (c->heads < 1 || c->d % c->heads ||
         !(c->d / c->heads == 16 || c->d / c->heads == 32 || c->d / c->heads == 64))
       return fail(nullptr, OCCU_EINVAL, "Graphormer: d / heads must be 16, 32 or 64");
@@ -323,6 +323,12 @@ occu_status forward(occu_ctx *ctx, const DevCsr &csr, const float *nf, const flo
     }
   }
   const float *h_top = w.h[c.L - 1].as<float>();
+  if (bf && (gph || dec)) {
+    // R41: in OCCU_BF16 the Graphormer layers / the decoder run in FP32 on the BF16-stored h_L
+    CK(w.hf.ensure(size_t(csr.N) * c.d * 4), "alloc FP32 h_L");
+    LK(launch_bf16_to_f32(ctx, w.h[c.L - 1].ptr, size_t(csr.N) * c.d, w.hf.as<float>(), s), "h_L to FP32");
+    h_top = w.hf.as<float>();
+  }
   if (gph) {
     // NEXT-3: Graphormer layers over each graph's node set (ping-pong between two buffers)
     if (w.gh.size() < size_t(c.graphormer)) w.gh.resize(c.graphormer);

@@ -154,8 +154,7 @@ def test_graphormer_errors():
     for bad in (dict(G=5, heads=4), dict(G=1, heads=16), dict(G=1, heads=3)):
         with pytest.raises(occu.OccuError):
             occu.Model(mk(2, 128, **bad))
-    with pytest.raises(occu.OccuError):
-        occu.Model(occu.config(L=2, d=64, prec=occu.BF16, graphormer=1, heads=2))
+    occu.Model(occu.config(L=2, d=64, prec=occu.BF16, graphormer=1, heads=2))     # R41: valid
     m = occu.Model(mk(2, 64, 1, 2))
     m.init_weights(1)
     with pytest.raises(occu.OccuError):
@@ -187,3 +186,27 @@ def test_graphormer_cfg3_sized_graphs():
     c = mk(3, 128, 1, 4)
     b = configs.cfg3(512).subset([0, 300])
     check(c, b, params_for(c, 31))
+
+
+@pytest.mark.parametrize("G,readout", [(2, 0), (2, 1), (0, 1)])
+def test_bf16_anee_with_fp32_graphormer_and_decoder(G, readout):
+    """OCCU_BF16 (R41): BF16 ANEE rounds, then the Graphormer layers / the decoder in FP32 on
+    the BF16-stored h_L.  Layer outputs vs oracle.forward_bf16 (same roundings) within the
+    mode's 1e-2; ŷ vs the float64 oracle at the BF16 criterion (R25)."""
+    c = occu.config(L=3, F_n=80, F_e=4, d=128, prec=occu.BF16, readout=readout, k=2, heads=4,
+                    graphormer=G)
+    b = configs.random_dag_batch(20, 2400 + G + readout, max_nodes=120, hub=True)
+    flat = params_for(c, 17)
+    m = occu.Model(c)
+    m.set_params(flat)
+    y = m.predict(occu.pack(b.graphs), b.node_feat, b.edge_feat)
+    params = oracle.unflatten(ocfg(c), flat.astype(np.float64))
+    pk = oracle.pack(b.graphs)
+    emu = oracle.forward_bf16(params, ocfg(c), pk, b.node_feat, b.edge_feat)
+    for j in range(G):
+        got = m.get_tensor(occu.T_GPH, j, (b.num_nodes, c.d))
+        assert rel(got, emu["gph"][j]) <= 1e-2, (j, rel(got, emu["gph"][j]))
+    assert rel(y, emu["yhat"]) <= 1e-2
+    yr = oracle.forward(params, ocfg(c), pk, b.node_feat, b.edge_feat)["yhat"]
+    assert rel(y, yr) <= 1e-2
+    assert np.all(np.abs(y - yr) <= 1e-2 * np.maximum(np.abs(yr), 0.1)), np.abs(y - yr).max()
