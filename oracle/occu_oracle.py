@@ -313,7 +313,9 @@ def forward_bf16(params, cfg, pk, node_feat, edge_feat, rnd=None):
         # R41: Graphormer layers / the decoder run in FP32 on the BF16-stored last h
         f = dict(layers=layers, h0=np.asarray(node_feat, np.float64),
                  e0=np.asarray(edge_feat, np.float64)[pk["in_eid"].astype(np.int64)])
-        return readout_stack(params, cfg, pk, f, layers[-1]["h"])
+        # R42: the Graphormer attention takes one fp16 product per step in this mode
+        return readout_stack(params, cfg, pk, f, layers[-1]["h"],
+                             att_rnd=fp16_round if rnd is None else rnd)
     n_b = np.diff(pk["node_off"].astype(np.int64))
     r = segment_sum(layers[-1]["h_f32"], pk["node_graph"].astype(np.int64), pk["num_graphs"]) / n_b[:, None]
     c = r @ params["W_1"].T + params["b_1"]                       # P125 (R12)
@@ -344,8 +346,10 @@ def ffn(x, params, p):
     return np.maximum(x @ params[p + "W1"].T + params[p + "b1"], 0.0) @ params[p + "W2"].T + params[p + "b2"]
 
 
-def mha(X, Y, params, m, heads):
-    """Multi-head attention MHA(X, Y, Y): queries from X, keys and values from Y."""
+def mha(X, Y, params, m, heads, rnd=None):
+    """Multi-head attention MHA(X, Y, Y): queries from X, keys and values from Y.  rnd (OCCU_BF16
+    Graphormer attention, R42): the operands of the two products — Q·log2(e)/√d_h, K, V and the
+    unnormalised weights 2^(s - max) — are rounded by rnd; the normaliser is the unrounded sum."""
     Q = X @ params[m + "Wq"].T + params[m + "bq"]
     K = Y @ params[m + "Wk"].T + params[m + "bk"]
     V = Y @ params[m + "Wv"].T + params[m + "bv"]
@@ -353,8 +357,13 @@ def mha(X, Y, params, m, heads):
     out = np.zeros_like(Q)
     for h in range(heads):
         sl = slice(h * dh, (h + 1) * dh)
-        A = softmax_channels(Q[:, sl] @ K[:, sl].T / np.sqrt(dh))     # softmax over the keys
-        out[:, sl] = A @ V[:, sl]
+        if rnd is None:
+            A = softmax_channels(Q[:, sl] @ K[:, sl].T / np.sqrt(dh))     # softmax over the keys
+            out[:, sl] = A @ V[:, sl]
+        else:
+            S = rnd(Q[:, sl] * (np.log2(np.e) / np.sqrt(dh))) @ rnd(K[:, sl]).T
+            Pu = np.exp2(S - S.max(axis=1, keepdims=True))
+            out[:, sl] = (rnd(Pu) @ rnd(V[:, sl])) / Pu.sum(axis=1, keepdims=True)
     return out @ params[m + "Wo"].T + params[m + "bo"]
 
 
@@ -371,18 +380,23 @@ def set_decoder(H, params, heads):
     return ffn(sab, params, "D_")
 
 
-def graphormer_layer(H, params, j, heads):
+def fp16_round(x):
+    """Round to the nearest IEEE fp16 (ties to even)."""
+    return np.asarray(x, np.float64).astype(np.float16).astype(np.float64)
+
+
+def graphormer_layer(H, params, j, heads, att_rnd=None):
     """Graphormer layer j over one graph's node states H [n, d] (P153-P157; R35-R37):
         h̄ = MHA(LN(h)) + h,    h' = FFN(LN(h̄)) + h̄
     with self-attention over all n nodes of the graph (MHA(X, X, X), R32 heads)."""
     g = f"G{j}_"
     X = layer_norm(H, params[g + "ln1_g"], params[g + "ln1_b"])
-    Hb = mha(X, X, params, g, heads) + H
+    Hb = mha(X, X, params, g, heads, att_rnd) + H
     Y = layer_norm(Hb, params[g + "ln2_g"], params[g + "ln2_b"])
     return ffn(Y, params, g + "F_") + Hb
 
 
-def readout_stack(params, cfg, pk, f, hL):
+def readout_stack(params, cfg, pk, f, hL, att_rnd=None):
     """cfg["graphormer"] Graphormer layers per graph (NEXT-3) on the last ANEE states hL, then
     the readout — the segmented mean (a7) or, with cfg["readout"] == 1, the Set-Transformer
     decoder per graph (NEXT-2) — and the MLP head on the (flattened) readout; fills f."""
@@ -390,7 +404,7 @@ def readout_stack(params, cfg, pk, f, hL):
     B = pk["num_graphs"]
     gph = []
     for j in range(cfg.get("graphormer", 0)):
-        hL = np.concatenate([graphormer_layer(hL[off[b]:off[b + 1]], params, j, cfg["heads"])
+        hL = np.concatenate([graphormer_layer(hL[off[b]:off[b + 1]], params, j, cfg["heads"], att_rnd)
                              for b in range(B)])
         gph.append(hL)
     f["gph"] = gph

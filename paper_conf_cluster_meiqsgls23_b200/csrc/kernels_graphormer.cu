@@ -586,6 +586,8 @@ __device__ __forceinline__ void fence_proxy_async_smem() {
   asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
 }
 
+// SPLIT = false (OCCU_BF16, R42): one fp16 product per step (Q, K, V, P rounded to fp16).
+template <bool SPLIT>
 __global__ void __launch_bounds__(128, 4) gph_attn_tc_kernel(const AttnArgs a) {
   using namespace gtc;
   extern __shared__ __align__(1024) uint8_t gsm_raw[];
@@ -686,9 +688,14 @@ __global__ void __launch_bounds__(128, 4) gph_attn_tc_kernel(const AttnArgs a) {
 #pragma unroll
       for (int kk = 0; kk < 2; ++kk) {
         const uint64_t bh = tc::sdesc_sw128(kh_a + kk * 32), bl = tc::sdesc_sw128(kl_a + kk * 32);
-        tc::mma_f16_ts(tmem + SC, tmem + QL + kk * 8, bh, id_s, kk > 0 ? 1u : 0u);
-        tc::mma_f16_ts(tmem + SC, tmem + QH + kk * 8, bl, id_s, 1u);
-        tc::mma_f16_ts(tmem + SC, tmem + QH + kk * 8, bh, id_s, 1u);
+        if constexpr (SPLIT) {
+          tc::mma_f16_ts(tmem + SC, tmem + QL + kk * 8, bh, id_s, kk > 0 ? 1u : 0u);
+          tc::mma_f16_ts(tmem + SC, tmem + QH + kk * 8, bl, id_s, 1u);
+          tc::mma_f16_ts(tmem + SC, tmem + QH + kk * 8, bh, id_s, 1u);
+        } else {
+          (void)bl;
+          tc::mma_f16_ts(tmem + SC, tmem + QH + kk * 8, bh, id_s, kk > 0 ? 1u : 0u);
+        }
       }
       tc::mma_commit(bar);
     }
@@ -728,7 +735,7 @@ __global__ void __launch_bounds__(128, 4) gph_attn_tc_kernel(const AttnArgs a) {
           split_h2(p0, p1, ph[j], pl[j]);
         }
         tc::tmem_st16(lane_base + PH + 16 * hf, ph);
-        tc::tmem_st16(lane_base + PL + 16 * hf, pl);
+        if constexpr (SPLIT) tc::tmem_st16(lane_base + PL + 16 * hf, pl);
       }
       l = l * f + sum;
       if (__any_sync(0xffffffffu, f != 1.f)) {     // rescale the O row (warp-collective)
@@ -748,8 +755,12 @@ __global__ void __launch_bounds__(128, 4) gph_attn_tc_kernel(const AttnArgs a) {
 #pragma unroll
       for (int kk = 0; kk < 4; ++kk) {
         const uint64_t bh = tc::sdesc_sw128(vh_a + kk * 32), bl = tc::sdesc_sw128(vl_a + kk * 32);
-        tc::mma_f16_ts(tmem + OC, tmem + PL + kk * 8, bh, id_o, 1u);
-        tc::mma_f16_ts(tmem + OC, tmem + PH + kk * 8, bl, id_o, 1u);
+        if constexpr (SPLIT) {
+          tc::mma_f16_ts(tmem + OC, tmem + PL + kk * 8, bh, id_o, 1u);
+          tc::mma_f16_ts(tmem + OC, tmem + PH + kk * 8, bl, id_o, 1u);
+        } else {
+          (void)bl;
+        }
         tc::mma_f16_ts(tmem + OC, tmem + PH + kk * 8, bh, id_o, 1u);
       }
       tc::mma_commit(bar);
@@ -834,9 +845,14 @@ int launch_graphormer_layer(const occu_ctx *ctx, const DevCsr &csr, int j, const
     return !e || atoi(e) != 0;
   }();
   if (use_tc && dh == 32 && !tf32) {    // tcgen05 path (d_h = 32)
-    cudaFuncSetAttribute(gph_attn_tc_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, int(gtc::SMEM));
     const dim3 g2((N + 127) / 128, cf.heads);
-    gph_attn_tc_kernel<<<g2, 128, gtc::SMEM, st>>>(a);
+    if (cf.prec == OCCU_BF16) {         // R42: one fp16 product per step
+      cudaFuncSetAttribute(gph_attn_tc_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, int(gtc::SMEM));
+      gph_attn_tc_kernel<false><<<g2, 128, gtc::SMEM, st>>>(a);
+    } else {
+      cudaFuncSetAttribute(gph_attn_tc_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, int(gtc::SMEM));
+      gph_attn_tc_kernel<true><<<g2, 128, gtc::SMEM, st>>>(a);
+    }
   } else if (tf32) {       // A/B: the TF32-split variant
     switch (dh) {
       case 16: go(gph_attn_kernel<16>, 16); break;

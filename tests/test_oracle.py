@@ -858,3 +858,19 @@ def test_forward_bf16_reading_b_identity_rounding_and_chain_closed_form():
         lay = fc["layers"][i]
         assert np.array_equal(lay["g"], np.ones_like(lay["g"]))
         assert np.allclose(lay["h_f32"][1:], oracle.leaky_relu(lay["hbar"][:5], cfg["slope"]), rtol=1e-15, atol=0)
+
+
+def test_mha_fp16_rounded_variant_limits():
+    """R42: with the identity as rounding the fp16-operand MHA is the plain MHA (same
+    function); with fp16 rounding it stays within fp16's relative precision of it."""
+    rng = np.random.default_rng(3)
+    d, heads = 16, 4
+    p = {f"G_W{w}": rng.standard_normal((d, d)) / 4 for w in "qkvo"}
+    p.update({f"G_b{w}": rng.standard_normal(d) / 4 for w in "qkvo"})
+    X = rng.standard_normal((11, d))
+    ref = oracle.mha(X, X, p, "G_", heads)
+    assert np.allclose(oracle.mha(X, X, p, "G_", heads, rnd=lambda x: np.asarray(x, np.float64)), ref,
+                       rtol=1e-12, atol=1e-13)
+    r16 = oracle.mha(X, X, p, "G_", heads, rnd=oracle.fp16_round)
+    assert np.linalg.norm(r16 - ref) <= 4e-3 * np.linalg.norm(ref)
+    assert not np.array_equal(r16, ref)
