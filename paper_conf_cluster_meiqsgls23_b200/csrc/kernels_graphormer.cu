@@ -341,6 +341,10 @@ __device__ __forceinline__ void split_h2(float x0, float x1, uint32_t &hi, uint3
   hi = *reinterpret_cast<const uint32_t *>(&h);
   lo = *reinterpret_cast<const uint32_t *>(&l);
 }
+__device__ __forceinline__ uint32_t pack_h2(float x0, float x1) {
+  const __half2 h = __floats2half2_rn(x0, x1);
+  return *reinterpret_cast<const uint32_t *>(&h);
+}
 __device__ __forceinline__ void ldsm_x4(uint32_t addr, uint32_t (&r)[4]) {
   asm volatile("ldmatrix.sync.aligned.m8n8.x4.shared.b16 {%0,%1,%2,%3}, [%4];"
                : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]) : "r"(addr));
@@ -666,19 +670,31 @@ __global__ void __launch_bounds__(128, 4) gph_attn_tc_kernel(const AttnArgs a) {
       uint32_t h[8], lw[8];
 #pragma unroll
       for (int c = 0; c < 4; ++c) {
-        split_h2(kx[c].x, kx[c].y, h[2 * c], lw[2 * c]);
-        split_h2(kx[c].z, kx[c].w, h[2 * c + 1], lw[2 * c + 1]);
+        if constexpr (SPLIT) {
+          split_h2(kx[c].x, kx[c].y, h[2 * c], lw[2 * c]);
+          split_h2(kx[c].z, kx[c].w, h[2 * c + 1], lw[2 * c + 1]);
+        } else {
+          h[2 * c] = pack_h2(kx[c].x, kx[c].y);
+          h[2 * c + 1] = pack_h2(kx[c].z, kx[c].w);
+        }
       }
       *reinterpret_cast<uint4 *>(Kh + tc::sw128_offset_f16(kr, d0, KB)) = make_uint4(h[0], h[1], h[2], h[3]);
       *reinterpret_cast<uint4 *>(Kh + tc::sw128_offset_f16(kr, d0 + 8, KB)) = make_uint4(h[4], h[5], h[6], h[7]);
-      *reinterpret_cast<uint4 *>(Kl + tc::sw128_offset_f16(kr, d0, KB)) = make_uint4(lw[0], lw[1], lw[2], lw[3]);
-      *reinterpret_cast<uint4 *>(Kl + tc::sw128_offset_f16(kr, d0 + 8, KB)) = make_uint4(lw[4], lw[5], lw[6], lw[7]);
+      if constexpr (SPLIT) {
+        *reinterpret_cast<uint4 *>(Kl + tc::sw128_offset_f16(kr, d0, KB)) = make_uint4(lw[0], lw[1], lw[2], lw[3]);
+        *reinterpret_cast<uint4 *>(Kl + tc::sw128_offset_f16(kr, d0 + 8, KB)) = make_uint4(lw[4], lw[5], lw[6], lw[7]);
+      }
 #pragma unroll
-      for (int c = 0; c < 8; ++c) split_h2(vx[2 * c], vx[2 * c + 1], h[c], lw[c]);
+      for (int c = 0; c < 8; ++c) {
+        if constexpr (SPLIT) split_h2(vx[2 * c], vx[2 * c + 1], h[c], lw[c]);
+        else h[c] = pack_h2(vx[2 * c], vx[2 * c + 1]);
+      }
       *reinterpret_cast<uint4 *>(Vh + tc::sw128_offset_f16(lane, vk0, 32)) = make_uint4(h[0], h[1], h[2], h[3]);
       *reinterpret_cast<uint4 *>(Vh + tc::sw128_offset_f16(lane, vk0 + 8, 32)) = make_uint4(h[4], h[5], h[6], h[7]);
-      *reinterpret_cast<uint4 *>(Vl + tc::sw128_offset_f16(lane, vk0, 32)) = make_uint4(lw[0], lw[1], lw[2], lw[3]);
-      *reinterpret_cast<uint4 *>(Vl + tc::sw128_offset_f16(lane, vk0 + 8, 32)) = make_uint4(lw[4], lw[5], lw[6], lw[7]);
+      if constexpr (SPLIT) {
+        *reinterpret_cast<uint4 *>(Vl + tc::sw128_offset_f16(lane, vk0, 32)) = make_uint4(lw[0], lw[1], lw[2], lw[3]);
+        *reinterpret_cast<uint4 *>(Vl + tc::sw128_offset_f16(lane, vk0 + 8, 32)) = make_uint4(lw[4], lw[5], lw[6], lw[7]);
+      }
     }
     fence_proxy_async_smem();
     tc::fence_before_sync();
@@ -732,7 +748,8 @@ __global__ void __launch_bounds__(128, 4) gph_attn_tc_kernel(const AttnArgs a) {
           const float p0 = ex2f(__uint_as_float(src[2 * j]) - ref);
           const float p1 = ex2f(__uint_as_float(src[2 * j + 1]) - ref);
           sum += p0 + p1;
-          split_h2(p0, p1, ph[j], pl[j]);
+          if constexpr (SPLIT) split_h2(p0, p1, ph[j], pl[j]);
+          else ph[j] = pack_h2(p0, p1);
         }
         tc::tmem_st16(lane_base + PH + 16 * hf, ph);
         if constexpr (SPLIT) tc::tmem_st16(lane_base + PL + 16 * hf, pl);
