@@ -44,7 +44,8 @@ struct SynthGraph {       // per graph of the batch (uploaded per call)
   float hp[4];            // batch, cin, seq, hw
 };
 
-__device__ __forceinline__ float enc(double x) { return float(log2(1.0 + x) / 40.0); }
+// log2(1 + 0) / 40 = 0 exactly: the many zero quantities (unused operator-hp slots) skip the log
+__device__ __forceinline__ float enc(double x) { return x == 0.0 ? 0.f : float(log2(1.0 + x) / 40.0); }
 
 __device__ __forceinline__ void newton_basis(const float *hp, double (&bv)[NC]) {
   const double nb[2] = {1.0, double(hp[0]) - BN0};
