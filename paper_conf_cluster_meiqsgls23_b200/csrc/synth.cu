@@ -27,7 +27,8 @@ struct occu_template {
   void *dmem;               // one device allocation holding everything below
   const int32_t *in_ptr, *in_src, *in_dst, *in_eid, *out_ptr, *out_pos;
   const float *nstatic, *estatic;   // [n][80], [m][4]
-  const double *ncoef, *ecoef;      // [n][22][12], [m][12]
+  const uint32_t *code;             // [n·22 + m] sparse polynomial codes: (start << 12) | mask
+  const double *coef;               // packed non-zero Newton coefficients
 };
 
 namespace occu {
@@ -39,7 +40,8 @@ constexpr double BN0 = 4.0, CN0 = 1.0, SN0 = 16.0, SN1 = 32.0;   // Newton nodes
 struct SynthGraph {       // per graph of the batch (uploaded per call)
   const int32_t *in_ptr, *in_src, *in_dst, *in_eid, *out_ptr, *out_pos;
   const float *nstatic, *estatic;
-  const double *ncoef, *ecoef;
+  const uint32_t *code;     // sparse polynomials: node quantities [n][22], then edges [m]
+  const double *coef;
   int32_t n, m, node_off, edge_off;
   float hp[4];            // batch, cin, seq, hw
 };
@@ -60,10 +62,15 @@ __device__ __forceinline__ void newton_basis(const float *hp, double (&bv)[NC]) 
       for (int k = 0; k < 3; ++k) bv[i * 6 + j * 3 + k] = nb[i] * nc[j] * ns[k];
 }
 
-__device__ __forceinline__ double poly(const double *__restrict__ c, const double (&bv)[NC]) {
+// Sparse Newton form: bit mi of the code's low 12 bits marks a non-zero coefficient mi; the
+// non-zeros are packed from index code >> 12 on.  Summed in coefficient order — the skipped
+// terms are exact zeros, so the result equals the dense sum.
+__device__ __forceinline__ double poly(uint32_t code, const double *__restrict__ c, const double (&bv)[NC]) {
   double q = 0.0;
+  uint32_t idx = code >> 12;
 #pragma unroll
-  for (int mi = 0; mi < NC; ++mi) q += __ldg(c + mi) * bv[mi];     // coefficient order (exact)
+  for (int mi = 0; mi < NC; ++mi)
+    if (code & (1u << mi)) q += __ldg(c + idx++) * bv[mi];
   return q;
 }
 
@@ -112,7 +119,7 @@ __global__ void __launch_bounds__(ST) synth_kernel(const SynthGraph *__restrict_
     in_dst[e0 + k] = n0 + __ldg(g.in_dst + k);
     in_eid[e0 + k] = e0 + __ldg(g.in_eid + k);
     out_pos[e0 + k] = e0 + __ldg(g.out_pos + k);
-    const double x = poly(g.ecoef + size_t(k) * NC, bv);
+    const double x = poly(__ldg(g.code + size_t(n) * NQ + k), g.coef, bv);
     const size_t er = size_t(e0 + k) * FE;
     *reinterpret_cast<float4 *>(ef + er) =
         make_float4(__ldg(g.estatic + size_t(k) * FE), __ldg(g.estatic + size_t(k) * FE + 1), enc(x),
@@ -121,7 +128,7 @@ __global__ void __launch_bounds__(ST) synth_kernel(const SynthGraph *__restrict_
   if (t < 4) cfgv[t] = enc(double(g.hp[t]));
   for (int i = t; i < un * NQ; i += ST) {        // the 22 quantities of the slice's nodes
     const int r = i / NQ, q = i % NQ;
-    const double x = poly(g.ncoef + (size_t(u0 + r) * NQ + q) * NC, bv);
+    const double x = poly(__ldg(g.code + size_t(u0 + r) * NQ + q), g.coef, bv);
     qv[r][q] = enc(x);
     if (q >= 16 && q < 20) qv[r][NQ + (q - 16)] = enc(4.0 * x);     // bytes = 4 x size
   }
@@ -172,12 +179,30 @@ extern "C" occu_status occu_template_create(occu_ctx *ctx, const occu_graph_view
   occu_status st = occu_pack(graph, 1, &h);      // validates the graph (ids, self-loops)
   if (st != OCCU_OK) return fail(ctx, st, std::string("occu_template_create: ") + global_error());
   const size_t n = size_t(graph->num_nodes), m = size_t(graph->num_edges);
-  // layout (bytes): ints [in_ptr n+1 | out_ptr n+1 | in_src m | in_dst m | in_eid m | out_pos m],
-  // then (8-aligned) doubles [ncoef n·22·12 | ecoef m·12], floats [nstatic n·80 | estatic m·4]
-  const size_t ni = 2 * (n + 1) + 4 * m;
+  // sparse polynomial codes: (start << 12) | non-zero mask, node quantities then edges
+  std::vector<uint32_t> codes(n * NQ + m);
+  std::vector<double> packed;
+  for (size_t pi = 0; pi < n * NQ + m; ++pi) {
+    const double *c = pi < n * NQ ? node_coef + pi * NC : edge_coef + (pi - n * NQ) * NC;
+    uint32_t mask = 0;
+    const size_t start = packed.size();
+    for (int mi = 0; mi < NC; ++mi)
+      if (c[mi] != 0.0) {
+        mask |= 1u << mi;
+        packed.push_back(c[mi]);
+      }
+    if (start >= (size_t(1) << 20)) {
+      occu_batch_free(h);
+      return fail(ctx, OCCU_EINVAL, "occu_template_create: more than 2^20 non-zero coefficients");
+    }
+    codes[pi] = uint32_t(start << 12) | mask;
+  }
+  // layout (bytes): ints [in_ptr n+1 | out_ptr n+1 | in_src m | in_dst m | in_eid m | out_pos m |
+  // codes n·22+m], then (16-aligned) doubles [packed non-zeros], floats [nstatic n·80 | estatic m·4]
+  const size_t ni = 2 * (n + 1) + 4 * m + codes.size();
   const size_t off_d = ((ni * 4 + 15) / 16) * 16;
-  const size_t nd = n * NQ * NC + m * NC;
-  const size_t off_f = off_d + nd * 8;
+  const size_t nd = packed.size();
+  const size_t off_f = off_d + ((nd * 8 + 15) / 16) * 16;
   const size_t total = off_f + (n * FN + m * FE) * 4;
   std::vector<unsigned char> hbuf(total, 0);
   int32_t *ip = reinterpret_cast<int32_t *>(hbuf.data());
@@ -188,8 +213,8 @@ extern "C" occu_status occu_template_create(occu_ctx *ctx, const occu_graph_view
   memcpy(ip + 2 * (n + 1) + 2 * m, h->in_eid, m * 4);
   memcpy(ip + 2 * (n + 1) + 3 * m, h->out_pos, m * 4);
   occu_batch_free(h);
-  memcpy(hbuf.data() + off_d, node_coef, n * NQ * NC * 8);
-  if (m) memcpy(hbuf.data() + off_d + n * NQ * NC * 8, edge_coef, m * NC * 8);
+  memcpy(ip + 2 * (n + 1) + 4 * m, codes.data(), codes.size() * 4);
+  if (nd) memcpy(hbuf.data() + off_d, packed.data(), nd * 8);
   memcpy(hbuf.data() + off_f, node_static, n * FN * 4);
   if (m) memcpy(hbuf.data() + off_f + n * FN * 4, edge_static, m * FE * 4);
   CK(cudaSetDevice(ctx->device), "cudaSetDevice");
@@ -213,8 +238,8 @@ extern "C" occu_status occu_template_create(occu_ctx *ctx, const occu_graph_view
   t->in_eid = t->in_dst + m;
   t->out_pos = t->in_eid + m;
   const unsigned char *db = static_cast<const unsigned char *>(d);
-  t->ncoef = reinterpret_cast<const double *>(db + off_d);
-  t->ecoef = t->ncoef + n * NQ * NC;
+  t->code = reinterpret_cast<const uint32_t *>(t->out_pos + m);
+  t->coef = reinterpret_cast<const double *>(db + off_d);
   t->nstatic = reinterpret_cast<const float *>(db + off_f);
   t->estatic = t->nstatic + n * FN;
   *out = t;
@@ -248,7 +273,7 @@ extern "C" occu_status occu_synthesize(occu_ctx *ctx, const occu_template *const
     SynthGraph &g = gs[b];
     g.in_ptr = t->in_ptr; g.in_src = t->in_src; g.in_dst = t->in_dst; g.in_eid = t->in_eid;
     g.out_ptr = t->out_ptr; g.out_pos = t->out_pos;
-    g.nstatic = t->nstatic; g.estatic = t->estatic; g.ncoef = t->ncoef; g.ecoef = t->ecoef;
+    g.nstatic = t->nstatic; g.estatic = t->estatic; g.code = t->code; g.coef = t->coef;
     g.n = t->n; g.m = t->m;
     g.node_off = int32_t(N);
     g.edge_off = int32_t(E);
