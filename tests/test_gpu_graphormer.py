@@ -188,13 +188,13 @@ def test_graphormer_cfg3_sized_graphs():
     check(c, b, params_for(c, 31))
 
 
-@pytest.mark.parametrize("G,readout", [(2, 0), (2, 1), (0, 1)])
-def test_bf16_anee_with_fp32_graphormer_and_decoder(G, readout):
+@pytest.mark.parametrize("G,readout,msg", [(2, 0, 0), (2, 1, 0), (0, 1, 0), (1, 1, 1)])
+def test_bf16_anee_with_fp32_graphormer_and_decoder(G, readout, msg):
     """OCCU_BF16 (R41): BF16 ANEE rounds, then the Graphormer layers / the decoder in FP32 on
     the BF16-stored h_L.  Layer outputs vs oracle.forward_bf16 (same roundings) within the
     mode's 1e-2; ŷ vs the float64 oracle at the BF16 criterion (R25)."""
     c = occu.config(L=3, F_n=80, F_e=4, d=128, prec=occu.BF16, readout=readout, k=2, heads=4,
-                    graphormer=G)
+                    graphormer=G, msg=msg)
     b = configs.random_dag_batch(20, 2400 + G + readout, max_nodes=120, hub=True)
     flat = params_for(c, 17)
     m = occu.Model(c)
