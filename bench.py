@@ -1081,6 +1081,14 @@ def main():
             "clocks": dict(clk.summary(), window="warm-up + timed region + 0.5 s continuation"),
             "roofline": roof,
             "aggregation": agg,
+            "tensor_pipe": {"what": "ncu sm__pipe_tensor_cycles_active % per GEMM kernel (profiles/"
+                                    "traffic*.json, cold-cache serialised replays); these GEMMs are "
+                                    "HBM-bound at d = 128 (DESIGN.md §6)",
+                            "f32": {k_: v_.get("tensor_pipe_pct") for k_, v_ in traffic.items()
+                                    if v_.get("tensor_pipe_pct")},
+                            "next_rows": {k_: v_.get("tensor_pipe_pct")
+                                          for k_, v_ in load_traffic("traffic_next.json").items()
+                                          if v_.get("tensor_pipe_pct")}},
             "kernel_ms_per_step": {k: v["ms_per_step"] for k, v in kernels.items()},
             "kernels": kernels,
             "kernel_timing": {"how": "CUDA events around every library launch (on its stream) "
