@@ -136,7 +136,7 @@ __device__ void warp_gemv_bf(const float *__restrict__ W, int ldw, int ncols, in
     }
     const int q = lane / NV, v = lane % NV, n = n0 + q;
     if (v < nvec && n < nrows) {
-      const float a = val[0] + (bias ? __ldg(bias + n) : 0.f);
+      const float a = val[0] + (bias ? bias[n] : 0.f);      // bias: global or shared
       Y[v * ldy + n] = relu ? fmaxf(a, 0.f) : a;
     }
   }
@@ -177,7 +177,7 @@ __device__ void warp_add_ln(const float *A, const float *Bv, float *Y, int nvec,
 #pragma unroll
     for (int i = 0; i < V; ++i) {
       const int ch = lane + 32 * i;
-      Y[v * D + ch] = (x[i] - mu) * inv * __ldg(g + ch) + __ldg(b + ch);
+      Y[v * D + ch] = (x[i] - mu) * inv * g[ch] + b[ch];   // g, b: global or shared
     }
   }
 }
@@ -527,9 +527,11 @@ __global__ void __launch_bounds__(DT) set_decoder_pool_mma_kernel(const DecArgs 
 // row read from L2 once per CTA serves GPC graphs).
 constexpr int GPC = 1;
 constexpr int DT_TAIL = 256;   // tail CTA: 8 warps (all B CTAs resident at once)
+constexpr int NPV = 20;         // the tail's bias / LayerNorm vectors
 template <int D>
 constexpr size_t tail_smem_floats(int d_h) {
-  return size_t(GPC) * (KMAX * KMAX * 8 + KHMAX * D + 6 * KMAX * D + SPLIT * KHMAX + KHMAX + d_h);
+  return size_t(GPC) * (KMAX * KMAX * 8 + KHMAX * D + 6 * KMAX * D + SPLIT * KHMAX + KHMAX + d_h) +
+         size_t(NPV) * D + size_t(KMAX) * D;
 }
 
 template <int D>
@@ -547,12 +549,22 @@ __global__ void __launch_bounds__(DT_TAIL) set_decoder_kernel(const DecArgs a, c
   float *fs = B5 + BS;                       // [GPC][SPLIT][KHMAX] partial scale factors
   float *lsum = fs + GPC * SPLIT * KHMAX;    // [GPC][KHMAX]
   float *cvec = lsum + GPC * KHMAX;          // [GPC][d_h]
+  float *pv = cvec + GPC * a.d_h;            // [NPV][D] biases / LayerNorm vectors, then S [k][D]
   const int t = threadIdx.x;
-  const float *P = a.P;
   const DecLayout &L = a.L;
   const float isq = rsqrtf(float(dh));
   pdl_trigger();
   pdl_wait();
+  {   // every small parameter vector of the chain into shared memory at once (one L2 latency)
+    const size_t vo[NPV] = {L.M1.bv, L.M1.bo, L.M1.ln1_g, L.M1.ln1_b, L.M1.F.b1, L.M1.F.b2,
+                            L.M1.ln2_g, L.M1.ln2_b, L.M2.bq, L.M2.bk, L.M2.bv, L.M2.bo,
+                            L.M2.ln1_g, L.M2.ln1_b, L.M2.F.b1, L.M2.F.b2, L.M2.ln2_g, L.M2.ln2_b,
+                            L.D.b1, L.D.b2};
+    for (int i = t; i < NPV * D; i += DT_TAIL) pv[i] = __ldg(a.P + vo[i / D] + i % D);
+    for (int i = t; i < k * D; i += DT_TAIL) pv[NPV * D + i] = __ldg(a.P + L.S + i);
+  }
+  const float *P = a.P;
+  auto PV = [&](int i) -> const float * { return pv + i * D; };
   constexpr int PS = part_stride<D>();
   for (int o = t; o < G * KH; o += DT_TAIL) {     // global max, factors 2^{(m_s - M)·log2e}, total sum
     const int gg = o / KH, kh = o % KH;
@@ -581,24 +593,24 @@ __global__ void __launch_bounds__(DT_TAIL) set_decoder_kernel(const DecArgs a, c
   // ---- MAB1 = PMA_k: O = W_v P + b_v per head, X1 = W_o O + b_o, H̄ = LN(S + X1), LN(H̄ + FFN(H̄))
   for (int h = 0; h < heads; ++h)
     gemv_k(P + L.M1.Wv + long(h) * dh * D, D, D, dh, Pacc + h * D, heads * D, V, B0 + h * dh, D,
-              P + L.M1.bv + h * dh, false);
+              PV(0) + h * dh, false);
   __syncthreads();
-  gemv_k(P + L.M1.Wo, D, D, D, B0, D, V, B1, D, P + L.M1.bo, false);
-  for (int i = t; i < V * D; i += DT_TAIL) B3[i] = P[L.S + i % (k * D)];
+  gemv_k(P + L.M1.Wo, D, D, D, B0, D, V, B1, D, PV(1), false);
+  for (int i = t; i < V * D; i += DT_TAIL) B3[i] = pv[NPV * D + i % (k * D)];
   __syncthreads();
-  warp_add_ln<D>(B3, B1, B2, V, P + L.M1.ln1_g, P + L.M1.ln1_b);      // B2 = H̄1
+  warp_add_ln<D>(B3, B1, B2, V, PV(2), PV(3));      // B2 = H̄1
   __syncthreads();
-  gemv_k(P + L.M1.F.W1, D, D, D, B2, D, V, B3, D, P + L.M1.F.b1, true);
+  gemv_k(P + L.M1.F.W1, D, D, D, B2, D, V, B3, D, PV(4), true);
   __syncthreads();
-  gemv_k(P + L.M1.F.W2, D, D, D, B3, D, V, B4, D, P + L.M1.F.b2, false);
+  gemv_k(P + L.M1.F.W2, D, D, D, B3, D, V, B4, D, PV(5), false);
   __syncthreads();
-  warp_add_ln<D>(B2, B4, B5, V, P + L.M1.ln2_g, P + L.M1.ln2_b);      // B5 = PMA_k(Z)
+  warp_add_ln<D>(B2, B4, B5, V, PV(6), PV(7));      // B5 = PMA_k(Z)
   __syncthreads();
 
   // ---- MAB2 = SAB over each graph's k vectors
-  gemv_k(P + L.M2.Wq, D, D, D, B5, D, V, B0, D, P + L.M2.bq, false);
-  gemv_k(P + L.M2.Wk, D, D, D, B5, D, V, B1, D, P + L.M2.bk, false);
-  gemv_k(P + L.M2.Wv, D, D, D, B5, D, V, B2, D, P + L.M2.bv, false);
+  gemv_k(P + L.M2.Wq, D, D, D, B5, D, V, B0, D, PV(8), false);
+  gemv_k(P + L.M2.Wk, D, D, D, B5, D, V, B1, D, PV(9), false);
+  gemv_k(P + L.M2.Wv, D, D, D, B5, D, V, B2, D, PV(10), false);
   __syncthreads();
   const int HKK = heads * k * k;
   for (int o = t; o < G * HKK; o += DT_TAIL) {     // scores per (graph, head, query, key)
@@ -629,21 +641,21 @@ __global__ void __launch_bounds__(DT_TAIL) set_decoder_kernel(const DecArgs a, c
     B3[o] = acc;
   }
   __syncthreads();
-  gemv_k(P + L.M2.Wo, D, D, D, B3, D, V, B4, D, P + L.M2.bo, false);
+  gemv_k(P + L.M2.Wo, D, D, D, B3, D, V, B4, D, PV(11), false);
   __syncthreads();
-  warp_add_ln<D>(B5, B4, B0, V, P + L.M2.ln1_g, P + L.M2.ln1_b);      // B0 = H̄2
+  warp_add_ln<D>(B5, B4, B0, V, PV(12), PV(13));      // B0 = H̄2
   __syncthreads();
-  gemv_k(P + L.M2.F.W1, D, D, D, B0, D, V, B1, D, P + L.M2.F.b1, true);
+  gemv_k(P + L.M2.F.W1, D, D, D, B0, D, V, B1, D, PV(14), true);
   __syncthreads();
-  gemv_k(P + L.M2.F.W2, D, D, D, B1, D, V, B2, D, P + L.M2.F.b2, false);
+  gemv_k(P + L.M2.F.W2, D, D, D, B1, D, V, B2, D, PV(15), false);
   __syncthreads();
-  warp_add_ln<D>(B0, B2, B3, V, P + L.M2.ln2_g, P + L.M2.ln2_b);      // B3 = SAB(PMA_k(Z))
+  warp_add_ln<D>(B0, B2, B3, V, PV(16), PV(17));      // B3 = SAB(PMA_k(Z))
   __syncthreads();
 
   // ---- final FFN -> decoder output [k][D] per graph (flattened into r), then the head
-  gemv_k(P + L.D.W1, D, D, D, B3, D, V, B4, D, P + L.D.b1, true);
+  gemv_k(P + L.D.W1, D, D, D, B3, D, V, B4, D, PV(18), true);
   __syncthreads();
-  gemv_k(P + L.D.W2, D, D, D, B4, D, V, B5, D, P + L.D.b2, false);
+  gemv_k(P + L.D.W2, D, D, D, B4, D, V, B5, D, PV(19), false);
   __syncthreads();
   for (int i = t; i < V * D; i += DT_TAIL) a.r[long(g0) * k * D + i] = B5[i];
   warp_gemv(P + a.W_1, k * D, k * D, a.d_h, B5, k * D, G, cvec, a.d_h, P + a.b_1, false);
