@@ -6,6 +6,9 @@ data-parallel across the GPUs of one box, with an NCCL gradient allreduce";
   ranks by work w_g = N_g + E_g, ties broken by graph index then
   rank; each shard keeps the caller's graph order.
 * ``contiguous_shard``: work-balanced contiguous ranges (inference, CFG5).
+* ``gather_and_pack``: graph-sharded inference's optional collection step (SURVEY §8(e),
+  NEXT-4): every rank holds the predictions of its contiguous range; they are all-gathered in
+  rank order (= global graph order) and rank 0 runs the occu-packing consumer on them.
 * ``DataParallel``: one process per GPU; rank 0 asks the library for an NCCL
   unique id, torch.distributed broadcasts it, every rank calls occu_dist_init;
   ``train_step`` packs the local shard and calls occu_train_step with the
@@ -82,3 +85,29 @@ class DataParallel:
         csr = occu.pack(local.graphs)
         return self.model.train_step(csr, local.node_feat, local.edge_feat, local.targets, lr,
                                      global_num_graphs=batch.num_graphs)
+
+
+def gather_and_pack(local_pred, rank: int, world: int, pg=None, capacity: float = 1.0):
+    """All-gather every rank's predictions (contiguous shards, rank order = graph order) and
+    run occu-packing (occu_pack_jobs, P390-P392) on rank 0.  Returns (all predictions, slot of
+    each job, slot loads) on rank 0 and (all predictions, None, None) elsewhere."""
+    import torch
+    from . import occu
+    local = torch.as_tensor(np.ascontiguousarray(local_pred, dtype=np.float32))
+    if world > 1:
+        import torch.distributed as dist
+        pg = pg or dist
+        sizes = [torch.zeros(1, dtype=torch.int64) for _ in range(world)]
+        pg.all_gather(sizes, torch.tensor([local.numel()], dtype=torch.int64))
+        mx = int(max(int(x.item()) for x in sizes))
+        buf = torch.zeros(mx, dtype=torch.float32)
+        buf[:local.numel()] = local
+        parts = [torch.zeros(mx, dtype=torch.float32) for _ in range(world)]
+        pg.all_gather(parts, buf)
+        allp = np.concatenate([parts[r][:int(sizes[r].item())].numpy() for r in range(world)])
+    else:
+        allp = local.numpy()
+    if rank != 0:
+        return allp, None, None
+    slots, loads = occu.pack_jobs(allp, capacity)
+    return allp, slots, loads

@@ -71,3 +71,38 @@ def test_dp_gloo_world2_matches_full_batch():
     assert all(p.exitcode == 0 for p in procs)
     err = q.get(timeout=5)
     assert err < 1e-12, err
+
+
+def _infer_worker(rank, world, port, q):
+    import torch.distributed as tdist
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    tdist.init_process_group("gloo", rank=rank, world_size=world)
+    rng = np.random.default_rng(11)
+    work = rng.integers(10, 500, size=37)
+    preds = rng.random(37).astype(np.float32)          # stand-in for each graph's prediction
+    lo, hi = dist.contiguous_shard(work, world)[rank]
+    allp, slots, loads = dist.gather_and_pack(preds[lo:hi], rank, world)
+    if rank == 0:
+        ref_slots, ref_loads = dist.gather_and_pack(preds, 0, 1)[1:]
+        q.put((bool(np.array_equal(allp, preds)), bool(np.array_equal(slots, ref_slots)),
+               bool(np.array_equal(loads, ref_loads))))
+    tdist.barrier()
+    tdist.destroy_process_group()
+
+
+def test_sharded_inference_gather_and_pack_gloo_world2():
+    """Graph-sharded inference (contiguous work-balanced ranges, no collective on the data
+    path) plus the optional rank-0 collection: the all-gathered predictions are the global
+    vector in graph order and rank 0's occu-packing equals single-process packing."""
+    import torch.multiprocessing as mp
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = 30500 + (os.getpid() % 1000)
+    procs = [ctx.Process(target=_infer_worker, args=(r, 2, port, q)) for r in range(2)]
+    for p in procs:
+        p.start()
+    for p in procs:
+        p.join(120)
+    assert all(p.exitcode == 0 for p in procs)
+    assert q.get(timeout=5) == (True, True, True)
