@@ -383,3 +383,31 @@ def test_predict_async_pipeline_matches_predict():
     with pytest.raises(occu.OccuError):
         m.predict_async(occu.pack(b.graphs), torch.from_numpy(b.node_feat).to(dev),
                         torch.from_numpy(b.edge_feat).to(dev), torch.empty(b.num_graphs, device=dev))
+
+
+def test_cfg5_mixture_launch_sampled_graphs():
+    """BASELINE CFG5's launch unit: 1,024 graphs of the 20-family mixture (1.4 M nodes) on
+    device buffers, FP32 and OCCU_BF16; one sampled graph of every family present checked
+    against the oracle (FP32 at 1e-4, BF16 at the R25 criterion)."""
+    import torch
+    b = configs.mixture(1024, 1004)
+    params_f = None
+    for prec in (occu.FP32, occu.BF16):
+        c = occu.config(L=3, F_n=80, F_e=4, d=128, prec=prec)
+        flat = weights.unit_scale(wcfg(c), weights.init_flat(wcfg(c), 42))
+        m = occu.Model(c)
+        m.set_params(flat)
+        csr = m.to_device(occu.pack(b.graphs))
+        y = m.predict(csr, torch.from_numpy(b.node_feat).cuda(), torch.from_numpy(b.edge_feat).cuda())
+        torch.cuda.synchronize()
+        y = y.cpu().numpy()
+        params_f = oracle.unflatten(ocfg(c), flat.astype(np.float64))
+        seen = {}
+        for gi, fam in enumerate(b.families):
+            seen.setdefault(fam, gi)
+        assert len(seen) >= 15
+        for fam, gi in seen.items():
+            s = b.subset([gi])
+            yr = oracle.predict(params_f, ocfg(c), s.graphs, s.node_feat, s.edge_feat)[0]
+            tol = TOL * max(abs(yr), 1e-2) if prec == occu.FP32 else 1e-2 * max(abs(yr), 0.1)
+            assert abs(y[gi] - yr) <= tol, (fam, prec, y[gi], yr)
