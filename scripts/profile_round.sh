@@ -10,8 +10,8 @@ timeout 900 ncu --set full --clock-control none --import-source on \
   -k regex:"rowgemm|gather_segsum|edge_small" -s 7 -c 7 -o gpurun_out/prof_full \
   python scripts/prof_driver.py --steps 2 > gpurun_out/prof_full.log 2>&1
 echo "full rc=$?" >> gpurun_out/prof_full.log
-timeout 900 ncu --set full --clock-control none --import-source on \
-  -k regex:"rowgemm_kernel<128, [45]>|wgrad_tc|split_reduce|node_bwd" -s 12 -c 8 -o gpurun_out/prof_train \
+timeout 900 ncu --set full --clock-control none --import-source on --kernel-name-base demangled \
+  -k regex:"rowgemm_kernel<\(int\)128, \(int\)[45]>|wgrad_tc|split_reduce|node_bwd" -s 12 -c 8 -o gpurun_out/prof_train \
   python scripts/prof_driver.py --steps 3 --train > gpurun_out/prof_train.log 2>&1
 echo "train rc=$?" >> gpurun_out/prof_train.log
 timeout 900 ncu --set full --clock-control none --import-source on \

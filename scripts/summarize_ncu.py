@@ -6,7 +6,7 @@ out = os.environ.get("PROFILES_OUT", os.path.join(ROOT, "profiles"))
 os.makedirs(out, exist_ok=True)
 
 def kname(full):
-    m = re.search(r"rowgemm(?:_bf16)?_kernel<(\d+), (\d+)", full)
+    m = re.search(r"rowgemm(?:_bf16)?_kernel<(?:\(int\))?(\d+), (?:\(int\))?(\d+)", full)
     if m:
         return ["node_tc", "edge_tc", "gate_tc", "plain_tc", "gatebwd_tc", "edgebwd_tc",
                 "gateagg_tc"][int(m.group(2))]
