@@ -121,3 +121,20 @@ def test_feature_templates_exact_for_every_family():
         templates.verify(t, [configs.mixture_variant(fam, r) for _ in range(2)])
         assert t.node_coef.shape == (t.num_nodes, 22, 12)
         assert np.all(t.node_static[:, 42:76] == 0)
+
+
+def test_feature_template_verify_rejects_a_non_polynomial_quantity():
+    """templates.verify is a real check: perturbing one coefficient (a quantity that the
+    Newton form no longer reproduces) is reported."""
+    from occu_gen import templates
+    t = templates.build_template("lenet5")
+    t.node_coef[3, 20, 1] += 1.0                 # FLOPs of node 3: wrong batch slope
+    with pytest.raises(ValueError):
+        templates.verify(t, [{"batch": 24, "cin": 2}])
+
+
+def test_feature_template_hp_vector_defaults():
+    from occu_gen import templates
+    assert list(templates.hp_vector("resnet50", {"batch": 20, "cin": 3})) == [20.0, 3.0, 0.0, 0.0]
+    assert list(templates.hp_vector("lstm", {"batch": 128, "seq": 32})) == [128.0, 1.0, 32.0, 0.0]
+    assert list(templates.hp_vector("gpt2", {"batch": 16, "cin": 3, "seq": 512})) == [16.0, 3.0, 512.0, 0.0]
