@@ -50,15 +50,37 @@ class Batch:
                      self.targets[list(idx)].copy(), [self.families[i] for i in idx])
 
 
+_TEACHER_NORM = {}
+
+
+def _teacher_norm(seed: int, w: np.ndarray):
+    """(mean, std) of the teacher's linear score u = mean(X)·w over a fixed reference set:
+    the 21 families at their default hyperparameters (A100).  Fixed constants per seed, so a
+    graph's label never depends on the batch it is drawn in."""
+    if seed not in _TEACHER_NORM:
+        us = []
+        for fam in dags.FAMILIES:
+            hp = dags.default_hp(fam)
+            g = dags.training_graph(fam, hp)
+            X, _ = node_edge_features(g, hp, "A100")
+            us.append(float(X.astype(np.float64).mean(axis=0) @ w))
+        _TEACHER_NORM[seed] = (float(np.mean(us)), float(np.std(us)) or 1.0)
+    return _TEACHER_NORM[seed]
+
+
 def teacher_targets(node_feat_list, seed: int) -> np.ndarray:
-    """Synthetic labels: sigmoid of a seeded linear function of mean node features.
+    """Synthetic labels: sigmoid of a seeded, standardised linear function of mean node
+    features, y = σ(2·(u − μ)/σ_u) with u = mean(X)·w (μ, σ_u fixed per seed, see
+    ``_teacher_norm``), so labels spread over (0, 1) across families and variants.
 
     Stands in for profiled occupancy (P85-P95), which needs the paper's GPUs.
     """
     w = 2.0 * uniform01(seed, F_N) - 1.0
+    mu, sd = _teacher_norm(seed, w)
     ys = []
     for X in node_feat_list:
-        z = 4.0 * float(X.astype(np.float64).mean(axis=0) @ w)
+        u = float(X.astype(np.float64).mean(axis=0) @ w)
+        z = 2.0 * (u - mu) / sd
         ys.append(1.0 / (1.0 + np.exp(-z)))
     return np.asarray(ys, np.float32)
 
@@ -165,3 +187,19 @@ def random_dag_batch(num_graphs: int, seed: int, max_nodes: int = 12, hub: bool 
     y = r.uniform(num_graphs).astype(np.float32) * 0.8 + 0.1
     return Batch(graphs, np.concatenate(nfs), np.concatenate(efs).reshape(-1, f_e), y,
                  ["random"] * num_graphs)
+
+
+def make(specs, seed: int):
+    """Batch of the graphs described by ``specs`` [(family, hp)] (e.g. one rank's shard of
+    ``mixture_specs``); labels from the teacher of ``seed`` as in ``mixture``."""
+    return _make(list(specs), seed=seed)
+
+
+def spec_work(specs) -> np.ndarray:
+    """Work w = N_g + E_g of each (family, hp) spec without building its features (a
+    family's topology does not depend on its hyperparameters, R39)."""
+    out = []
+    for fam, hp in specs:
+        g = dags.training_graph(fam, hp)
+        out.append(g.num_nodes + g.num_edges)
+    return np.asarray(out, np.int64)

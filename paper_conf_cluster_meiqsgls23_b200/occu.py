@@ -429,9 +429,11 @@ class Model:
         ef, _, k2 = _ptr(edge_feat)
         op, _, k3 = _ptr(out)
         _check(lib().occu_predict_async(self._ctx, csr._p, nf, ef, op), self._ctx)
-        # the previous call's inputs are free once this call returns; outputs until wait()
-        self._inflight = [x for x in self._inflight if x[0] is None] + [(csr, k1, k2, k3, node_feat, edge_feat, out)]
-        self._inflight = [(None, None, None, None, None, None, x[6]) for x in self._inflight[:-1]] + self._inflight[-1:]
+        # the previous calls' inputs are free once this call returns (the library waits for
+        # their H2D copies); every output stays referenced until wait() (its D2H may be in
+        # flight).  Strip the earlier entries to their outputs, then append this call in full.
+        self._inflight = ([(None, None, None, None, None, None, x[6]) for x in self._inflight]
+                          + [(csr, k1, k2, k3, node_feat, edge_feat, out)])
         return out
 
     def wait(self):
