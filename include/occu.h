@@ -227,8 +227,26 @@ occu_status occu_pack_jobs(const float *occ, int32_t num_jobs, double capacity,
                            int32_t *slot_of_job, double *slot_load, int32_t *num_slots);
 
 /* ---- data parallel (north_star: NCCL gradient allreduce over NVLink) ------ */
+/* One process per GPU.  occu_nccl_unique_id: rank 0 creates the 128-byte id, the caller
+ * broadcasts it (e.g. torch.distributed); every rank then calls occu_dist_init with its rank and
+ * the world size (world >= 1; world = 1 runs the same NCCL data plane on one GPU).  The
+ * communicator is created non-blocking; occu_train_step then sums the flat gradient (+ the
+ * loss) with ncclAllReduce over NVLink on the ctx stream before Adam, so every rank applies the
+ * same update (replicas stay bitwise equal).  Errors: OCCU_EINVAL (NULL, bad rank / world),
+ * OCCU_ENCCL (NCCL failure, or no progress within the timeout: the communicator is then
+ * aborted with ncclCommAbort and every later collective call fails with OCCU_ENCCL until
+ * occu_dist_init is called again). */
 occu_status occu_nccl_unique_id(void *out_128_bytes);
 occu_status occu_dist_init(occu_ctx *ctx, int rank, int world, const void *nccl_unique_id);
+/* Watchdog timeout in seconds for communicator setup and for every blocking wait on a step that
+ * contains a collective (default 600; 0 disables).  OCCU_EINVAL if seconds < 0. */
+occu_status occu_dist_set_timeout(occu_ctx *ctx, double seconds);
+/* Abort the communicator (ncclCommAbort), e.g. from a host watchdog after a peer died; safe to
+ * call from another host thread while a step is waiting. */
+occu_status occu_dist_abort(occu_ctx *ctx);
+/* Wait (host) until everything enqueued on the ctx stream has completed, polling NCCL for
+ * asynchronous errors; OCCU_ENCCL + abort on error or timeout. */
+occu_status occu_dist_sync(occu_ctx *ctx);
 
 /* ---- optimizer state (Adam m, v, t) --------------------------------------- */
 occu_status occu_save_state(const occu_ctx *ctx, const char *path);

@@ -138,6 +138,8 @@ struct occu_ctx {
   // data parallel
   ncclComm *comm = nullptr;
   int rank = 0, world = 1;
+  double nccl_timeout_s = 600.0;   // occu_dist_set_timeout: watchdog on NCCL progress (0 = none)
+  bool comm_aborted = false;       // set when the watchdog (or occu_dist_abort) aborted comm
   std::string err;
 };
 

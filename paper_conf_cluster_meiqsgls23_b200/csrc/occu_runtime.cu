@@ -5,6 +5,9 @@
 #include <stdio.h>
 #include <stdlib.h>
 #include <string.h>
+#include <sched.h>
+#include <time.h>
+#include <unistd.h>
 
 #include <algorithm>
 #include <string>
@@ -463,6 +466,62 @@ occu_status grads_impl(occu_ctx *ctx, const occu_batch *batch, const float *targ
   return OCCU_OK;
 }
 
+
+// ---- NCCL watchdog -------------------------------------------------------------------
+// The communicator is non-blocking (ncclConfig_t::blocking = 0): NCCL calls return at once
+// (possibly ncclInProgress) and progress / asynchronous errors are polled here, so a dead
+// peer or a stuck collective surfaces as OCCU_ENCCL after ctx->nccl_timeout_s instead of a
+// hang; the communicator is then aborted (ncclCommAbort) and dropped.
+double now_s() {
+  timespec t;
+  clock_gettime(CLOCK_MONOTONIC, &t);
+  return double(t.tv_sec) + 1e-9 * double(t.tv_nsec);
+}
+
+occu_status nccl_abort(occu_ctx *ctx, const std::string &why) {
+  if (ctx->comm) {
+    ncclCommAbort(ctx->comm);
+    ctx->comm = nullptr;
+  }
+  ctx->comm_aborted = true;
+  return fail(ctx, OCCU_ENCCL, why);
+}
+
+// Wait until the communicator has no NCCL call in progress (setup or an enqueue).
+occu_status nccl_settle(occu_ctx *ctx, const char *what) {
+  const double t0 = now_s();
+  for (;;) {
+    ncclResult_t st = ncclSuccess;
+    ncclResult_t r = ncclCommGetAsyncError(ctx->comm, &st);
+    if (r != ncclSuccess) return nccl_abort(ctx, std::string(what) + ": ncclCommGetAsyncError: " + ncclGetErrorString(r));
+    if (st == ncclSuccess) return OCCU_OK;
+    if (st != ncclInProgress) return nccl_abort(ctx, std::string(what) + ": " + ncclGetErrorString(st));
+    if (ctx->nccl_timeout_s > 0 && now_s() - t0 > ctx->nccl_timeout_s)
+      return nccl_abort(ctx, std::string(what) + ": timed out (ncclCommAbort)");
+    sched_yield();
+  }
+}
+
+// Host wait for the ctx stream; with a communicator, poll NCCL errors and the timeout.
+occu_status stream_wait(occu_ctx *ctx, const char *what) {
+  if (!ctx->comm) {
+    CK(cudaStreamSynchronize(ctx->stream), what);
+    return OCCU_OK;
+  }
+  const double t0 = now_s();
+  for (;;) {
+    cudaError_t e = cudaStreamQuery(ctx->stream);
+    if (e == cudaSuccess) return OCCU_OK;
+    if (e != cudaErrorNotReady) return cuda_fail(ctx, e, what);
+    ncclResult_t st = ncclSuccess;
+    if (ncclCommGetAsyncError(ctx->comm, &st) != ncclSuccess || (st != ncclSuccess && st != ncclInProgress))
+      return nccl_abort(ctx, std::string(what) + ": NCCL asynchronous error " + ncclGetErrorString(st));
+    if (ctx->nccl_timeout_s > 0 && now_s() - t0 > ctx->nccl_timeout_s)
+      return nccl_abort(ctx, std::string(what) + ": no progress within the timeout (ncclCommAbort)");
+    usleep(20);
+  }
+}
+
 }  // namespace
 
 // ============================================================================
@@ -731,10 +790,15 @@ occu_status occu_train_step(occu_ctx *ctx, const occu_batch *batch, const float 
   occu_status st = grads_impl(ctx, batch, targets, stg, csr);
   if (st != OCCU_OK) return st;
   const size_t n = ctx->layout.total + 1;
-  if (ctx->comm && ctx->world > 1) {
+  if (ctx->comm_aborted && !ctx->comm)
+    return fail(ctx, OCCU_ENCCL, "the communicator was aborted; call occu_dist_init again");
+  if (ctx->comm) {
+    // a11: sum of the flat gradient (+ loss slot) over the ranks, in place, on the ctx stream
     ncclResult_t r = ncclAllReduce(ctx->grads.ptr, ctx->grads.ptr, n, ncclFloat32, ncclSum,
                                    ctx->comm, ctx->stream);
-    if (r != ncclSuccess) return fail(ctx, OCCU_ENCCL, std::string("ncclAllReduce: ") + ncclGetErrorString(r));
+    if (r != ncclSuccess && r != ncclInProgress)
+      return nccl_abort(ctx, std::string("ncclAllReduce: ") + ncclGetErrorString(r));
+    if ((st = nccl_settle(ctx, "ncclAllReduce")) != OCCU_OK) return st;
   }
   ctx->adam_t += 1;
   LK(launch_adam(ctx, lr, ctx->stream), "adam");
@@ -742,7 +806,7 @@ occu_status occu_train_step(occu_ctx *ctx, const occu_batch *batch, const float 
     float l = 0.f;
     CK(cudaMemcpyAsync(&l, ctx->grads.as<float>() + ctx->layout.total, 4, cudaMemcpyDeviceToHost,
                        ctx->stream), "loss D2H");
-    CK(cudaStreamSynchronize(ctx->stream), "sync");
+    if ((st = stream_wait(ctx, "train step")) != OCCU_OK) return st;
     if (out_loss) *out_loss = l;
   }
   return OCCU_OK;
@@ -795,13 +859,39 @@ occu_status occu_dist_init(occu_ctx *ctx, int rank, int world, const void *nccl_
   }
   ncclUniqueId id;
   memcpy(&id, nccl_unique_id, 128);
-  ncclComm_t comm;
-  ncclResult_t r = ncclCommInitRank(&comm, world, id, rank);
-  if (r != ncclSuccess) return fail(ctx, OCCU_ENCCL, std::string("ncclCommInitRank: ") + ncclGetErrorString(r));
+  ncclConfig_t cfg = NCCL_CONFIG_INITIALIZER;
+  cfg.blocking = 0;                      // progress polled by the watchdog (nccl_settle)
+  ncclComm_t comm = nullptr;
+  ncclResult_t r = ncclCommInitRankConfig(&comm, world, id, rank, &cfg);
+  if (r != ncclSuccess && r != ncclInProgress) {
+    if (comm) ncclCommAbort(comm);
+    return fail(ctx, OCCU_ENCCL, std::string("ncclCommInitRankConfig: ") + ncclGetErrorString(r));
+  }
   ctx->comm = comm;
+  ctx->comm_aborted = false;
   ctx->rank = rank;
   ctx->world = world;
+  return nccl_settle(ctx, "ncclCommInitRankConfig");
+}
+
+occu_status occu_dist_set_timeout(occu_ctx *ctx, double seconds) {
+  if (!ctx) return fail(nullptr, OCCU_EINVAL, "ctx is NULL");
+  if (!(seconds >= 0.0)) return fail(ctx, OCCU_EINVAL, "timeout must be >= 0");
+  ctx->nccl_timeout_s = seconds;
   return OCCU_OK;
+}
+
+occu_status occu_dist_abort(occu_ctx *ctx) {
+  if (!ctx) return fail(nullptr, OCCU_EINVAL, "ctx is NULL");
+  if (!ctx->comm) return OCCU_OK;
+  nccl_abort(ctx, "aborted by occu_dist_abort");
+  return OCCU_OK;
+}
+
+occu_status occu_dist_sync(occu_ctx *ctx) {
+  if (!ctx) return fail(nullptr, OCCU_EINVAL, "ctx is NULL");
+  CK(cudaSetDevice(ctx->device), "cudaSetDevice");
+  return stream_wait(ctx, "occu_dist_sync");
 }
 
 occu_status occu_save_state(const occu_ctx *cctx, const char *path) {

@@ -33,6 +33,7 @@ EXPORTS = [
     "occu_get_tensor", "occu_last_launch_count", "occu_last_error", "occu_set_profiling",
     "occu_profile_reset", "occu_profile_query", "occu_set_kernel_path", "occu_pack_jobs",
     "occu_template_create", "occu_template_destroy", "occu_synthesize", "occu_set_small_batch_kernel",
+    "occu_dist_set_timeout", "occu_dist_abort", "occu_dist_sync",
 ]
 
 
@@ -106,6 +107,9 @@ def lib():
             "occu_set_weight_decay": ([VP, C.c_float], I32),
             "occu_nccl_unique_id": ([VP], I32),
             "occu_dist_init": ([VP, C.c_int, C.c_int, VP], I32),
+            "occu_dist_set_timeout": ([VP, C.c_double], I32),
+            "occu_dist_abort": ([VP], I32),
+            "occu_dist_sync": ([VP], I32),
             "occu_save_state": ([VP, C.c_char_p], I32),
             "occu_load_state": ([VP, C.c_char_p], I32),
             "occu_set_keep_intermediates": ([VP, C.c_int], I32),
@@ -472,6 +476,15 @@ class Model:
     def dist_init(self, rank: int, world: int, uid: bytes):
         buf = (C.c_ubyte * 128).from_buffer_copy(uid)
         _check(lib().occu_dist_init(self._ctx, rank, world, buf), self._ctx)
+
+    def dist_set_timeout(self, seconds: float):
+        _check(lib().occu_dist_set_timeout(self._ctx, float(seconds)), self._ctx)
+
+    def dist_abort(self):
+        _check(lib().occu_dist_abort(self._ctx), self._ctx)
+
+    def dist_sync(self):
+        _check(lib().occu_dist_sync(self._ctx), self._ctx)
 
     def set_kernel_path(self, path: int):
         """0 = tensor cores (default), 1 = CUDA-core SIMT FP32, 2 = tensor cores with the

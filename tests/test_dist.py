@@ -106,3 +106,20 @@ def test_sharded_inference_gather_and_pack_gloo_world2():
         p.join(120)
     assert all(p.exitcode == 0 for p in procs)
     assert q.get(timeout=5) == (True, True, True)
+
+
+def test_dataparallel_host_sharding_uses_global_batch():
+    """DataParallel packs only its LPT shard and scales by the GLOBAL batch size."""
+    b = configs.mixture(24, 1004)
+    seen = {}
+
+    class Fake:
+        def train_step(self, csr, nf, ef, y, lr, global_num_graphs=None):
+            seen["B"] = csr.num_graphs
+            seen["G"] = global_num_graphs
+            return 0.0
+
+    dp = dist.DataParallel(Fake(), 1, 3)
+    dp.train_step(b, 1e-3)
+    idx = dist.lpt_shard(dist.graph_work(b.graphs), 3)[1]
+    assert seen == {"B": len(idx), "G": 24}
