@@ -114,12 +114,23 @@ def test_dataparallel_host_sharding_uses_global_batch():
     seen = {}
 
     class Fake:
+        def nccl_unique_id(self):
+            return b"u" * 128
+
+        def dist_init(self, rank, world, uid):
+            seen["init"] = (rank, world, uid)
+
         def train_step(self, csr, nf, ef, y, lr, global_num_graphs=None):
             seen["B"] = csr.num_graphs
             seen["G"] = global_num_graphs
             return 0.0
 
-    dp = dist.DataParallel(Fake(), 1, 3)
+    class FakePG:                     # rank 0's id reaches every rank through the broadcast
+        @staticmethod
+        def broadcast_object_list(lst, src=0):
+            lst[0] = b"u" * 128
+
+    dp = dist.DataParallel(Fake(), 1, 3, pg=FakePG)
     dp.train_step(b, 1e-3)
     idx = dist.lpt_shard(dist.graph_work(b.graphs), 3)[1]
-    assert seen == {"B": len(idx), "G": 24}
+    assert seen == {"B": len(idx), "G": 24, "init": (1, 3, b"u" * 128)}
