@@ -457,30 +457,207 @@ def maxvit_t(b: Builder):
     return b.linear(x, 1000)
 
 
+# ---------------------------------------------------------------------------
+# BERT / GPT-2 as the paper's largest graphs (P239: up to 2,664 nodes): the torch.onnx export
+# of the Hugging Face modules in training mode under AMP autocast, constant folding off.
+# Relative to the compact ONNX-style blocks above this adds what such an export contains:
+# autocast Casts on every Linear operand (input, weight, bias) and around the fp32 ops
+# (Softmax, LayerNorm), opset-13+ axes / ratio / training-mode inputs as Constant nodes
+# (Unsqueeze, ReduceMean, Dropout), HF's `x.size()[:-1] + (...)` shape arithmetic
+# (Shape -> Slice -> Concat -> Reshape), GPT-2's Conv1D (view -> addmm -> view), its causal
+# mask slice (Shape / Gather / Sub / Slice / Where) per layer and its tanh GELU.  DESIGN.md R43.
+# ---------------------------------------------------------------------------
+class _HF:
+    def __init__(self, b: Builder):
+        self.b = b
+
+    def const(self):
+        return self.b.const()
+
+    def cast(self, x, shape=None):
+        return self.b.add("Cast", [x], self.b.shape(x) if shape is None else shape)
+
+    def unsq(self, x, shape):
+        return self.b.add("Unsqueeze", [x, self.const()], shape)
+
+    def slice_(self, x, shape):
+        # Slice(data, starts, ends, axes, steps)
+        return self.b.add("Slice", [x, self.const(), self.const(), self.const(), self.const()], shape)
+
+    def size_reshape(self, x, new_shape, keep):
+        """HF shape arithmetic: x.size()[:keep] + (extra...) -> Reshape."""
+        b = self.b
+        sh = b.add("Shape", [x], (len(b.shape(x)),))
+        head = self.slice_(sh, (keep,))
+        extra = [self.const() for _ in range(len(new_shape) - keep)]
+        cat = b.add("Concat", [head] + extra, (len(new_shape),))
+        return b.add("Reshape", [x, cat], new_shape)
+
+    def linear(self, x, out):
+        """nn.Linear under autocast: Cast(x), Cast(W), Cast(b) -> MatMul (transposed weight)
+        -> Add(bias)."""
+        b = self.b
+        s = b.shape(x)
+        k = s[-1]
+        xc = self.cast(x)
+        wc = b.add("Cast", [], (out, k), (), [(out, k)])
+        wt = b.add("Transpose", [wc], (k, out))
+        y = b.add("MatMul", [xc, wt], tuple(s[:-1]) + (out,), (k, out), (),
+                  2.0 * numel(s[:-1]) * out * k)
+        bc = b.add("Cast", [], (out,), (), [(out,)])
+        return b.add("Add", [y, bc], b.shape(y))
+
+    def conv1d(self, x, out):
+        """GPT-2 Conv1D: size_out = x.size()[:-1] + (nf,); x.view(-1, x.size(-1)) ->
+        addmm(bias, x, W) (Gemm) -> view(size_out); autocast Casts on the operands."""
+        b = self.b
+        s = b.shape(x)
+        k = s[-1]
+        m = numel(s[:-1])
+        sh = b.add("Shape", [x], (len(s),))
+        last = b.add("Gather", [sh, self.const()], (1,))
+        u = self.unsq(last, (1,))
+        cat = b.add("Concat", [self.const(), u], (2,))
+        flat = b.add("Reshape", [x, cat], (m, k))
+        xc = self.cast(flat)
+        wc = b.add("Cast", [], (k, out), (), [(k, out)])
+        bc = b.add("Cast", [], (out,), (), [(out,)])
+        g = b.add("Gemm", [bc, xc, wc], (m, out), (k, out), (), 2.0 * m * out * k)
+        sh2 = b.add("Shape", [x], (len(s),))
+        head = self.slice_(sh2, (len(s) - 1,))
+        cat2 = b.add("Concat", [head, self.const()], (len(s),))
+        return b.add("Reshape", [g, cat2], tuple(s[:-1]) + (out,))
+
+    def dropout(self, x):
+        # training-mode Dropout(data, ratio, training_mode) -> (output, mask)
+        return self.b.add("Dropout", [x, self.const(), self.const()], self.b.shape(x))
+
+    def layernorm(self, x):
+        """LayerNorm autocast to fp32, decomposed (opset < 17), axes as Constant inputs."""
+        b = self.b
+        s = b.shape(x)
+        h = s[-1]
+        red = tuple(s[:-1]) + (1,)
+        xf = self.cast(x)
+        m = b.add("ReduceMean", [xf, self.const()], red)
+        d = b.add("Sub", [xf, m], s)
+        p = b.add("Pow", [d, self.const()], s)
+        v = b.add("ReduceMean", [p, self.const()], red)
+        e = b.add("Add", [v, self.const()], red)
+        q = b.add("Sqrt", [e], red)
+        n = b.add("Div", [d, q], s)
+        g = b.add("Mul", [n], s, (), [(h,)])
+        return b.add("Add", [g], s, (), [(h,)])
+
+    def softmax(self, x):
+        xf = self.cast(x)
+        y = self.b.add("Softmax", [xf], self.b.shape(x), (), (), 5.0 * numel(self.b.shape(x)))
+        return self.cast(y)
+
+    def gelu_erf(self, x):
+        b = self.b
+        s = b.shape(x)
+        a = b.add("Div", [x, self.const()], s)
+        e = b.add("Erf", [a], s)
+        c = b.add("Add", [e, self.const()], s)
+        d = b.add("Mul", [x, c], s)
+        return b.add("Mul", [d, self.const()], s)
+
+    def gelu_tanh(self, x):
+        """gelu_new: 0.5·x·(1 + tanh(sqrt(2/π)·(x + 0.044715·x³)))."""
+        b = self.b
+        s = b.shape(x)
+        p3 = b.add("Pow", [x, self.const()], s)
+        m1 = b.add("Mul", [p3, self.const()], s)
+        a1 = b.add("Add", [x, m1], s)
+        m2 = b.add("Mul", [a1, self.const()], s)
+        t = b.add("Tanh", [m2], s)
+        a2 = b.add("Add", [t, self.const()], s)
+        m3 = b.add("Mul", [x, self.const()], s)
+        return b.add("Mul", [m3, a2], s)
+
+    def attention(self, x, heads, mask, causal):
+        b = self.b
+        n, t, h = b.shape(x)
+        dh = h // heads
+        if causal:                                  # c_attn: one Conv1D, then split
+            qkv = self.conv1d(x, 3 * h)
+            sp = b.add("Split", [qkv, self.const()], (n, t, h))
+            parts = [sp, b.add("Identity", [sp], (n, t, h)), b.add("Identity", [sp], (n, t, h))]
+        else:
+            parts = [self.linear(x, h) for _ in range(3)]
+        heads_ = []
+        for y in parts:
+            y = self.size_reshape(y, (n, t, heads, dh), 2)
+            heads_.append(b.add("Transpose", [y], (n, heads, t, dh)))
+        q, k, v = heads_
+        kt = b.add("Transpose", [k], (n, heads, dh, t))
+        sc = b.add("MatMul", [q, kt], (n, heads, t, t), (dh,), (), 2.0 * n * heads * t * t * dh)
+        sc = b.add("Div", [sc, self.const()], (n, heads, t, t))
+        if causal:                                  # bias[:, :, k-q:k, :k], torch.where(...)
+            shq = b.add("Shape", [q], (4,))
+            ql = b.add("Gather", [shq, self.const()], (1,))
+            shk = b.add("Shape", [k], (4,))
+            kl = b.add("Gather", [shk, self.const()], (1,))
+            st = b.add("Sub", [kl, ql], (1,))
+            s1 = b.add("Slice", [self.const(), self.unsq(st, (1,)), self.unsq(kl, (1,)),
+                                 self.const(), self.const()], (1, 1, t, 1024))
+            s2 = b.add("Slice", [s1, self.const(), self.unsq(kl, (1,)), self.const(), self.const()],
+                       (1, 1, t, t))
+            cm = b.add("Cast", [s2], (1, 1, t, t))
+            fill = b.add("Cast", [self.const()], (1,))
+            sc = b.add("Where", [cm, sc, fill], (n, heads, t, t))
+        sc = b.add("Add", [sc, mask], (n, heads, t, t))
+        pr = self.dropout(self.softmax(sc))
+        o = b.add("MatMul", [pr, v], (n, heads, t, dh), (t,), (), 2.0 * n * heads * t * t * dh)
+        o = b.add("Transpose", [o], (n, t, heads, dh))
+        o = self.size_reshape(o, (n, t, h), 2)
+        return self.conv1d(o, h) if causal else self.linear(o, h)
+
+    def block(self, x, heads, mask, causal):
+        b = self.b
+        h = b.shape(x)[-1]
+        if causal:                                   # GPT-2: pre-LN
+            y = self.attention(self.layernorm(x), heads, mask, True)
+            x = b.add2(x, self.dropout(y))
+            y = self.conv1d(self.gelu_tanh(self.conv1d(self.layernorm(x), 4 * h)), h)
+            return b.add2(x, self.dropout(y))
+        y = self.dropout(self.attention(x, heads, mask, False))
+        x = self.layernorm(b.add2(y, x))
+        y = self.dropout(self.linear(self.gelu_erf(self.linear(x, 4 * h)), h))
+        return self.layernorm(b.add2(y, x))
+
+
 def _bert(depth, dim, heads, causal=False):
     def build(b: Builder):
+        hf = _HF(b)
         n, t = b.hp["batch"], b.hp["seq"]
         ids = b.add("Identity", [], (n, t))
         sh = b.add("Shape", [ids], (2,))
-        ln_ = b.add("Gather", [sh], (1,))
-        pos = b.add("Slice", [ln_], (1, t))
+        ln_ = b.add("Gather", [sh, b.const()], (1,))
+        pos = hf.slice_(ln_, (1, t))
         tok = b.add("Gather", [ids], (n, t, dim), (), [(30522 if not causal else 50257, dim)])
         pe = b.add("Gather", [pos], (1, t, dim), (), [(512 if not causal else 1024, dim)])
         x = b.add2(tok, pe)
         if not causal:
-            x = b.layernorm(x)
-        mask = b.add("Cast", [b.add("Unsqueeze", [ids], (n, 1, 1, t))], (n, 1, 1, t))
-        mask = b.add("Mul", [b.add("Sub", [mask], (n, 1, 1, t))], (n, 1, 1, t))
-        if causal:
-            mask = b.add("Where", [mask], (n, 1, t, t))
+            tt = b.add("Gather", [b.add("Identity", [], (n, t))], (n, t, dim), (), [(2, dim)])
+            x = hf.dropout(hf.layernorm(b.add2(x, tt)))
+        else:
+            x = hf.dropout(x)
+        # extended attention mask: (1 - mask[:, None, None, :]) * finfo.min, in the model dtype
+        am = b.add("Identity", [], (n, t))
+        mask = hf.unsq(hf.unsq(am, (n, 1, t)), (n, 1, 1, t))
+        mask = hf.cast(mask)
+        mask = b.add("Sub", [b.const(), mask], (n, 1, 1, t))
+        mask = b.add("Mul", [mask, b.const()], (n, 1, 1, t))
         for _ in range(depth):
-            x = b.encoder_block(x, heads, pre_ln=causal, shape_ops=True)
+            x = hf.block(x, heads, mask, causal)
         if causal:
-            x = b.layernorm(x)
+            x = hf.layernorm(x)
             return b.linear(x, 50257, bias=False, op="MatMul")
-        x = b.add("Gather", [x], (n, dim))
-        x = b.add("Tanh", [b.linear(x, dim)], (n, dim))
-        return b.linear(x, 2)
+        x = b.add("Gather", [x, b.const()], (n, dim))
+        x = b.add("Tanh", [hf.linear(x, dim)], (n, dim))
+        return hf.linear(hf.dropout(x), 2)
     return build
 
 

@@ -548,19 +548,6 @@ def adam_step(params, grads, state, lr, wd=1e-4, beta1=0.9, beta2=0.999, eps=1e-
 
 
 # --------------------------------------------------------------------------
-# Metrics (P247-P253), used by examples/eval only.
-# --------------------------------------------------------------------------
-def mre(yhat, y):
-    yhat, y = np.asarray(yhat, np.float64), np.asarray(y, np.float64)
-    return float(np.mean(np.abs((yhat - y) / y)))
-
-
-def mse(yhat, y):
-    yhat, y = np.asarray(yhat, np.float64), np.asarray(y, np.float64)
-    return float(np.mean((yhat - y) ** 2))
-
-
-# --------------------------------------------------------------------------
 # NEXT-4 consumer: occu-packing (P390-P392; R38).  "an appropriate packing
 # policy for multiple jobs should ensure the cumulative occupancy is at most 100%" (P390);
 # "a GPU-occupancy-based bin-packing algorithm (with co-location ensuring GPU occupancy does

@@ -1326,14 +1326,16 @@ __global__ void __launch_bounds__(NT) node_bwd_kernel(
     const int32_t *__restrict__ in_ptr, int N, float slope, float *__restrict__ dP,
     float *__restrict__ dpq, float *__restrict__ da_part) {
   // da_part != null: also accumulate [da_s; da_d] = Σ_u [dp_u; dq_u] h̄_u per warp (fixed
-  // node assignment) into da_part[warp][2][D] for a fixed-order reduction.
+  // node assignment) into da_part[block][2][D] for a fixed-order reduction.  These sums
+  // cancel heavily (dp, dq and h̄ are signed), so they accumulate in float64.
   constexpr int V = D / 32;
   const int lane = threadIdx.x & 31;
   const int warps = (gridDim.x * NT) / 32;
-  float das[V], dad[V], a_sv[V], a_dv[V];
+  double das[V], dad[V];
+  float a_sv[V], a_dv[V];
 #pragma unroll
   for (int c = 0; c < V; ++c) {
-    das[c] = dad[c] = 0.f;
+    das[c] = dad[c] = 0.0;
     a_sv[c] = __ldg(a_s + lane * V + c);
     a_dv[c] = __ldg(a_d + lane * V + c);
   }
@@ -1380,8 +1382,8 @@ __global__ void __launch_bounds__(NT) node_bwd_kernel(
       const int ch = lane * V + c;
       const float v = acc[c] + dp * a_sv[c] + dq * a_dv[c];
       o[c] = v * lrelu_grad_from_out(hb[c], slope);
-      das[c] = fmaf(dp, hb[c], das[c]);
-      dad[c] = fmaf(dq, hb[c], dad[c]);
+      das[c] = fma(double(dp), double(hb[c]), das[c]);
+      dad[c] = fma(double(dq), double(hb[c]), dad[c]);
       (void)ch;
     }
     store_row<V>(dP + long(u) * D + lane * V, o);
@@ -1391,7 +1393,7 @@ __global__ void __launch_bounds__(NT) node_bwd_kernel(
     }
   }
   if (da_part) {   // per-block partial: warps combined in fixed warp order through smem
-    __shared__ float red[NT / 32][2 * D];
+    __shared__ double red[NT / 32][2 * D];
     const int wl = threadIdx.x / 32;
 #pragma unroll
     for (int c = 0; c < V; ++c) {
@@ -1400,9 +1402,9 @@ __global__ void __launch_bounds__(NT) node_bwd_kernel(
     }
     __syncthreads();
     for (int o = threadIdx.x; o < 2 * D; o += NT) {
-      float acc2 = 0.f;
+      double acc2 = 0.0;
       for (int w2 = 0; w2 < NT / 32; ++w2) acc2 += red[w2][o];
-      da_part[long(blockIdx.x) * 2 * D + o] = acc2;
+      da_part[long(blockIdx.x) * 2 * D + o] = float(acc2);
     }
   }
 }
@@ -1529,14 +1531,14 @@ struct ReduceJobs { ReduceJob j[4]; int blk[5]; int count; };
 // job.lanes threads per output (8 for 128x128 weight gradients, 64 for the few outputs of
 // [da_s; da_d] with thousands of partials), 256 / lanes outputs per block.
 __global__ void __launch_bounds__(256) multi_reduce_kernel(const ReduceJobs jobs) {
-  __shared__ float red[256];
+  __shared__ double red[256];   // partial sums of signed gradients cancel: float64
   int q = 0;
   while (q + 1 < jobs.count && int(blockIdx.x) >= jobs.blk[q + 1]) ++q;
   const ReduceJob jb = jobs.j[q];
   const int lanes = jb.lanes, opb = 256 / lanes;
   const int ol = threadIdx.x % opb, l = threadIdx.x / opb;
   const long o = long(int(blockIdx.x) - jobs.blk[q]) * opb + ol;
-  float a0 = 0.f, a1 = 0.f, a2 = 0.f, a3 = 0.f;     // four independent chains in flight
+  double a0 = 0.0, a1 = 0.0, a2 = 0.0, a3 = 0.0;     // four independent chains in flight
   if (o < jb.n) {
     int k = l;
     for (; k + 3 * lanes < jb.splits; k += 4 * lanes) {
@@ -1550,18 +1552,18 @@ __global__ void __launch_bounds__(256) multi_reduce_kernel(const ReduceJobs jobs
   red[l * opb + ol] = (a0 + a1) + (a2 + a3);
   __syncthreads();
   if (l == 0 && o < jb.n) {
-    float t = 0.f;
+    double t = 0.0;
     for (int x = 0; x < lanes; ++x) t += red[x * opb + ol];
-    jb.out[o] = t;
+    jb.out[o] = float(t);
   }
 }
 
 __global__ void wgrad_reduce_kernel(const float *__restrict__ partial, int splits, long n,
                                     float *__restrict__ out) {
   for (long i = blockIdx.x * long(blockDim.x) + threadIdx.x; i < n; i += long(gridDim.x) * blockDim.x) {
-    float s = 0.f;
+    double s = 0.0;
     for (int k = 0; k < splits; ++k) s += partial[long(k) * n + i];
-    out[i] = s;
+    out[i] = float(s);
   }
 }
 
@@ -2053,11 +2055,9 @@ static int backward_layer_impl(occu_ctx *ctx, const DevCsr &csr, const BwdLayerA
     ++n;
   }
   const int nb_blocks = grid_for(long(csr.N) * 32, NT, 16 * sms);
-  float *da_part = nullptr;
-  if (tc) {
-    if (w.dpart.ensure(size_t(nb_blocks) * 2 * D * 4) != cudaSuccess) return -int(cudaErrorMemoryAllocation);
-    da_part = w.dpart.as<float>();
-  }
+  // [da_s; da_d] partials from node_bwd on both kernel paths (float64 per block)
+  if (w.dpart.ensure(size_t(nb_blocks) * 2 * D * 4) != cudaSuccess) return -int(cudaErrorMemoryAllocation);
+  float *da_part = w.dpart.as<float>();
   OCCU_PROF_BEGIN(ctx, "node_bwd", st);
   if (bf)
     node_bwd_kernel<D, true><<<nb_blocks, NT, 0, st>>>(
@@ -2073,7 +2073,7 @@ static int backward_layer_impl(occu_ctx *ctx, const DevCsr &csr, const BwdLayerA
   // dW_m = DVᵀ E' ; dW_e = DZᵀ E_in ; dW_u = dPᵀ H_in ; [da_s; da_d] = [dp dq]ᵀ h̄ — partial
   // sums into per-GEMM slots, all of the layer's split reductions in one launch
   ReduceJobs rj{};
-  if (tc) rj.j[rj.count++] = ReduceJob{da_part, G + L.a_s[i], long(2 * D), nb_blocks};
+  rj.j[rj.count++] = ReduceJob{da_part, G + L.a_s[i], long(2 * D), nb_blocks};
   if (w.partial.ensure(3 * WG_SLOT_FLOATS * 4) != cudaSuccess) return -int(cudaErrorMemoryAllocation);
   float *slot = w.partial.as<float>();
   if ((r = wgrad_deferred(ctx, w.DV.as<float>(), D, a.e, D, csr.E, G + L.W_m[i], st, bf, rj, slot)) < 0) return r;
@@ -2086,10 +2086,6 @@ static int backward_layer_impl(occu_ctx *ctx, const DevCsr &csr, const BwdLayerA
   n += r;
   if ((r = launch_multi_reduce(ctx, rj, st)) < 0) return r;
   n += r;
-  if (!tc) {
-    if ((r = wgrad(ctx, w.dpq.as<float>(), 2, a.hbar, D, csr.N, G + L.a_s[i], st)) < 0) return r;
-    n += r;
-  }
   if (a.dh_prev && csr.N > 0 && tc) {   // dh^{i-1} = dP W_u on tensor cores
     if ((r = launch_plain_tc(ctx, w.dP.as<float>(), D, csr.N, 5, i, nullptr, a.dh_prev,
                              "dh_prev_tc", st, a.h_in, csr.in_ptr, in_bf)) < 0) return r;

@@ -13,7 +13,11 @@ from paper_conf_cluster_meiqsgls23_b200 import occu
 
 pytestmark = pytest.mark.gpu
 TOL = 1e-4
-GRAD_TOL = 2e-4
+GRAD_TOL = 1e-4          # per-tensor gradients: the FP32 tolerance (tensor-core paths)
+# The CUDA-core SIMT path (kernel path 1, opt-in, not the product default) is a second
+# implementation whose plain-FP32 GEMMs leave the cancellation-heavy first-layer a_s / a_d
+# gradients at 1.1e-4 through L = 3 unit-scale layers (R23): its own bound.
+GRAD_TOL_SIMT = 2e-4
 
 
 @pytest.fixture(scope="module", autouse=True)
@@ -55,17 +59,41 @@ def run_both(c, batch, flat, keep=True, path=0):
     return m, y, ref, pk
 
 
+def rows_ok(a, b, tol=TOL, what=""):
+    """Per-row check beside the tensor-wide rel-L2 (one wrong row of a large tensor is
+    diluted ~sqrt(rows) times in the tensor-wide norm): SURVEY Q19's relative-L2 criterion
+    applied to every row r, ||a_r - b_r||_2 <= tol * max(||b_r||_2, 1e-3 * max_r ||b_r||_2)
+    (the floor covers rows that are near-exact cancellations, e.g. sums of signed messages).
+    DESIGN.md R44 says why rows, not elements: e' = σ(α·z) amplifies the GEMM's rounding of
+    single channels by |α| where σ is steep."""
+    a = np.asarray(a, np.float64).reshape(len(b), -1)
+    b = np.asarray(b, np.float64).reshape(len(b), -1)
+    if b.size == 0:
+        return
+    err = np.linalg.norm(a - b, axis=1)
+    nb = np.linalg.norm(b, axis=1)
+    scale = np.maximum(nb, 1e-3 * nb.max())
+    scale = np.where(scale > 0, scale, 1.0)
+    bad = err > tol * scale
+    assert not bad.any(), (what, int(bad.sum()), int(np.argmax(err / scale)), float(np.max(err / scale)))
+
+
 def compare_all(m, c, y, ref, pk, tol=TOL):
     N, E, B, d = pk["num_nodes"], pk["num_edges"], pk["num_graphs"], c.d
     for i in range(c.L):
         lay = ref["layers"][i]
-        assert rel(m.get_tensor(occu.T_HBAR, i, (N, d)), lay["hbar"]) <= tol, ("hbar", i)
-        assert rel(m.get_tensor(occu.T_P, i, (N,)), lay["p"]) <= tol, ("p", i)
-        assert rel(m.get_tensor(occu.T_Q, i, (N,)), lay["q"]) <= tol, ("q", i)
-        if E:
-            assert rel(m.get_tensor(occu.T_E, i, (E, d)), lay["e"]) <= tol, ("e", i)
-        assert rel(m.get_tensor(occu.T_H, i, (N, d)), lay["h"]) <= tol, ("h", i)
-    assert rel(m.get_tensor(occu.T_R, 0, (B, d)), ref["r"]) <= tol
+        for name, t, shape, key in (("hbar", occu.T_HBAR, (N, d), "hbar"), ("p", occu.T_P, (N,), "p"),
+                                    ("q", occu.T_Q, (N,), "q"), ("e", occu.T_E, (E, d), "e"),
+                                    ("h", occu.T_H, (N, d), "h")):
+            if shape[0] == 0:
+                continue
+            got = m.get_tensor(t, i, shape)
+            assert rel(got, lay[key]) <= tol, (name, i, rel(got, lay[key]))
+            if len(shape) == 2:
+                rows_ok(got, lay[key], tol, (name, i))
+    r = m.get_tensor(occu.T_R, 0, (B, d))
+    assert rel(r, ref["r"]) <= tol
+    rows_ok(r, ref["r"], tol, "r")
     yr = ref["yhat"]
     assert np.all(np.abs(y - yr) <= tol * np.maximum(np.abs(yr), 1e-2)), np.abs(y - yr).max()
 
@@ -152,15 +180,17 @@ def test_cfg2_subset_unit_scale():
     compare_all(m, c, y, ref, pk)
 
 
-def test_cfg2_full_size_sampled_graphs():
-    """BASELINE CFG2 at full size (256 graphs) on device buffers, as bench.py runs
-    it; 6 sampled graphs checked one by one against the oracle."""
+def test_cfg2_full_size_every_graph_and_intermediate():
+    """BASELINE CFG2 at full size (256 ResNet-50 graphs, 131k nodes) on device buffers, as
+    bench.py runs it: all 256 ŷ and every intermediate (h̄, p, q, e', h per layer, r) against
+    the oracle's full-batch forward (rel-L2 and per-row checks)."""
     import torch
     c = mk(3, 128)
     b = configs.cfg2(256)
     flat = weights.unit_scale(wcfg(c), weights.init_flat(wcfg(c), 42))
     m = occu.Model(c)
     m.set_params(flat)
+    m.keep_intermediates(True)
     csr = m.to_device(occu.pack(b.graphs))
     nf = torch.from_numpy(b.node_feat).cuda()
     ef = torch.from_numpy(b.edge_feat).cuda()
@@ -168,10 +198,15 @@ def test_cfg2_full_size_sampled_graphs():
     torch.cuda.synchronize()
     y = y.cpu().numpy()
     params = oracle.unflatten(ocfg(c), flat.astype(np.float64))
-    for gi in (0, 1, 77, 128, 200, 255):
-        s = b.subset([gi])
-        yr = oracle.predict(params, ocfg(c), s.graphs, s.node_feat, s.edge_feat)
-        assert abs(y[gi] - yr[0]) <= TOL * max(abs(yr[0]), 1e-2), gi
+    pk = oracle.pack(b.graphs)
+    ref = oracle.forward(params, ocfg(c), pk, b.node_feat, b.edge_feat)
+    compare_all(m, c, y, ref, pk)
+    # the bench's launch configuration (no kept states: readout folded into the aggregation)
+    m.keep_intermediates(False)
+    y2 = m.predict(csr, nf, ef)
+    torch.cuda.synchronize()
+    yr = ref["yhat"]
+    assert np.all(np.abs(y2.cpu().numpy() - yr) <= TOL * np.maximum(np.abs(yr), 1e-2))
 
 
 @pytest.mark.parametrize("path", [0, 1, 2], ids=["tcgen05", "simt", "tcgen05fused"])
@@ -285,10 +320,11 @@ def test_gradients_match_oracle(L, d, aggr, path):
     params = oracle.unflatten(ocfg(c), flat.astype(np.float64))
     lref, gref = oracle.loss_and_grads(params, ocfg(c), b.graphs, b.node_feat, b.edge_feat, b.targets)
     assert abs(loss - lref) <= TOL * abs(lref)
+    tol = GRAD_TOL if path == 0 else GRAD_TOL_SIMT
     for k in gref:
-        # DESIGN.md R23: FP32 backward through 3 layers; the first-layer attention
-        # vectors' gradients are cancellation-heavy sums -> gradient tolerance 2e-4
-        assert rel(g[k], gref[k]) <= GRAD_TOL, (k, rel(g[k], gref[k]))
+        assert rel(g[k], gref[k]) <= tol, (k, rel(g[k], gref[k]))
+        if np.ndim(gref[k]) == 2:
+            rows_ok(g[k], gref[k], 10 * tol, k)
 
 
 def test_training_trajectory_matches_oracle():
@@ -325,7 +361,7 @@ def test_cfg3_full_size_training_properties():
     import torch
     c = mk(3, 128)
     b = configs.cfg3(512)
-    flat = weights.init_flat(wcfg(c), 42)
+    flat = weights.unit_scale(wcfg(c), weights.init_flat(wcfg(c), 42))   # ŷ varies (Q23)
     m = occu.Model(c)
     m.set_params(flat)
     dev = torch.device("cuda", 0)
@@ -343,6 +379,7 @@ def test_cfg3_full_size_training_properties():
         s = b.subset([gi])
         yr = oracle.predict(params, ocfg(c), s.graphs, s.node_feat, s.edge_feat)
         assert abs(y[gi] - yr[0]) <= TOL * max(abs(yr[0]), 1e-2), gi
+    assert np.std(y) > 1e-3 * max(np.abs(y).max(), 1e-6)      # not the vacuous ŷ ≈ b_2 regime
     loss = m.compute_grads(csr, nf, ef, yt)
     g_full = m.get_grads()
     want = float(np.mean((y - b.targets.astype(np.float64)) ** 2))
@@ -353,7 +390,9 @@ def test_cfg3_full_size_training_properties():
         hc, hn, he, hy = dev_batch(hb)
         m.compute_grads(hc, hn, he, hy, global_num_graphs=512)
         g_sum += m.get_grads().astype(np.float64)
-    assert rel(g_full, g_sum) <= 1e-5, rel(g_full, g_sum)
+    # two split-K partitions of the same sums: equal up to FP32 rounding (unit-scale weights
+    # make the sums cancellation-heavy), checked at the FP32 tolerance
+    assert rel(g_full, g_sum) <= TOL, rel(g_full, g_sum)
     # every parameter tensor receives a gradient (the identity above holds trivially for 0)
     for k, v in weights.unflatten(wcfg(c), g_full).items():
         assert np.linalg.norm(v) > 0, k
@@ -411,3 +450,57 @@ def test_cfg5_mixture_launch_sampled_graphs():
             yr = oracle.predict(params_f, ocfg(c), s.graphs, s.node_feat, s.edge_feat)[0]
             tol = TOL * max(abs(yr), 1e-2) if prec == occu.FP32 else 1e-2 * max(abs(yr), 0.1)
             assert abs(y[gi] - yr) <= tol, (fam, prec, y[gi], yr)
+
+
+def test_cfg3_slice_gradients_match_oracle():
+    """A 64-graph slice of CFG3 (32 BERT-base + 32 GPT-2 training graphs, ~190k nodes) with
+    unit-scale weights: loss and every per-tensor gradient against the float64 oracle."""
+    c = mk(3, 128)
+    full = configs.cfg3(512)
+    b = full.subset(list(range(0, 32)) + list(range(256, 288)))
+    flat = weights.unit_scale(wcfg(c), weights.init_flat(wcfg(c), 42))
+    m = occu.Model(c)
+    m.set_params(flat)
+    loss = m.compute_grads(occu.pack(b.graphs), b.node_feat, b.edge_feat, b.targets,
+                           global_num_graphs=512)
+    g = weights.unflatten(wcfg(c), m.get_grads())
+    params = oracle.unflatten(ocfg(c), flat.astype(np.float64))
+    lref, gref = oracle.loss_and_grads(params, ocfg(c), b.graphs, b.node_feat, b.edge_feat,
+                                       b.targets, global_batch=512)
+    assert abs(loss - lref) <= TOL * abs(lref)
+    for k in gref:
+        assert rel(g[k], gref[k]) <= GRAD_TOL, (k, rel(g[k], gref[k]))
+
+
+def test_save_and_load_state_resume_bitwise(tmp_path):
+    """occu_save_state / occu_load_state (+ the weights file) resume training exactly: a
+    model restored after 3 steps continues bitwise like the one that never stopped."""
+    c = mk(2, 64)
+    b = configs.random_dag_batch(20, 640, max_nodes=40, hub=True)
+    flat = weights.unit_scale(wcfg(c), weights.init_flat(wcfg(c), 13))
+    csr = occu.pack(b.graphs)
+    m = occu.Model(c)
+    m.set_params(flat)
+    for _ in range(3):
+        m.train_step(csr, b.node_feat, b.edge_feat, b.targets, 1e-3)
+    m.save_weights(str(tmp_path / "w.bin"))
+    m.save_state(str(tmp_path / "s.bin"))
+    m2 = occu.Model(c)
+    m2.load_weights(str(tmp_path / "w.bin"))
+    m2.load_state(str(tmp_path / "s.bin"))
+    for _ in range(3):
+        la = m.train_step(csr, b.node_feat, b.edge_feat, b.targets, 1e-3)
+        lb = m2.train_step(csr, b.node_feat, b.edge_feat, b.targets, 1e-3)
+        assert la == lb
+    assert np.array_equal(m.get_params(), m2.get_params())
+    # a fresh optimizer state (t = 0) takes a different step: the state file matters
+    m3 = occu.Model(c)
+    m3.load_weights(str(tmp_path / "w.bin"))
+    for _ in range(3):
+        m3.train_step(csr, b.node_feat, b.edge_feat, b.targets, 1e-3)
+    assert not np.array_equal(m3.get_params(), m.get_params())
+    # a state file of another configuration is rejected
+    m4 = occu.Model(mk(3, 64))
+    m4.init_weights(1)
+    with pytest.raises(occu.OccuError):
+        m4.load_state(str(tmp_path / "s.bin"))

@@ -14,7 +14,7 @@ from paper_conf_cluster_meiqsgls23_b200 import occu
 
 pytestmark = pytest.mark.gpu
 TOL = 1e-4
-GRAD_TOL = 2e-4
+GRAD_TOL = 1e-4
 MSGB = occu.MSG_NEIGHBOR_SOFTMAX
 
 
