@@ -203,3 +203,48 @@ def spec_work(specs) -> np.ndarray:
         g = dags.training_graph(fam, hp)
         out.append(g.num_nodes + g.num_edges)
     return np.asarray(out, np.int64)
+
+
+def mixture_arrays(num_graphs: int, seed: int, start: int = 0):
+    """Vectorised ``mixture_specs``: (family index into MIXTURE [num], hp [num, 4]) with hp the
+    ``templates.hp_vector`` row (batch, cin, seq, hw) of graph start .. start+num-1.  Same
+    counter-based draws as ``mixture_specs`` (stream (seed << 32) + k, outputs 1..4), for the
+    1M-graph CFG5 sweep and the 50k-graph CFG4 epoch (tests/test_gen.py checks the match)."""
+    from .prng import _GOLDEN, _M1, _M2
+    k = np.arange(start, start + num_graphs, dtype=np.uint64)
+    base = (np.uint64(seed) << np.uint64(32)) + k
+
+    def u(j):
+        with np.errstate(over="ignore"):
+            z = base + np.uint64(j) * _GOLDEN
+            z = (z ^ (z >> np.uint64(30))) * _M1
+            z = (z ^ (z >> np.uint64(27))) * _M2
+            z = z ^ (z >> np.uint64(31))
+        return (z >> np.uint64(11)).astype(np.float64) * (1.0 / 9007199254740992.0)
+
+    def ri(uu, lo, hi):
+        return lo + np.floor(uu * (hi - lo + 1))
+
+    u1, u2, u3, u4 = u(1), u(2), u(3), u(4)
+    fam = ri(u1, 0, len(MIXTURE) - 1).astype(np.int64)
+    kind = np.array([2 if f in dags.RNN else (1 if f in dags.TRANSFORMER else 0) for f in MIXTURE])[fam]
+    hp = np.zeros((num_graphs, 4), np.float64)
+    rnn, tr, cnn = kind == 2, kind == 1, kind == 0
+    hp[rnn, 0] = 8 * ri(u2[rnn], 16, 64)
+    hp[rnn, 1] = 1
+    hp[rnn, 2] = 8 * ri(u3[rnn], 2, 16)
+    hp[tr, 0] = 4 * ri(u2[tr], 4, 32)
+    hp[tr, 1] = ri(u3[tr], 1, 10)
+    hp[tr, 2] = np.where(ri(u4[tr], 0, 1) > 0, 512, 20)
+    hp[cnn, 0] = 4 * ri(u2[cnn], 4, 32)
+    hp[cnn, 1] = ri(u3[cnn], 1, 10)
+    return fam, hp
+
+
+def family_work() -> np.ndarray:
+    """N_g + E_g of each MIXTURE family's training DAG (topology is hp-independent)."""
+    out = []
+    for f in MIXTURE:
+        g = dags.training_graph(f, dags.default_hp(f))
+        out.append(g.num_nodes + g.num_edges)
+    return np.asarray(out, np.int64)

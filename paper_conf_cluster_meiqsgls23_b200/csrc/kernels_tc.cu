@@ -442,6 +442,15 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
       float aux = 0.f;
       if ((EPI == EPI_EDGE || EPI == EPI_EDGEBWD) && hf == 0 && live)
         aux = __ldg(a.pin + __ldg(a.src + r0 + row)) + __ldg(a.qin + __ldg(a.dst + r0 + row));  // α (R1)
+      // EDGEBWD: the row's first de chunk is fetched before waiting on the accumulator, and
+      // every later chunk one step ahead (the epilogue is paced by these per-row loads)
+      float4 dpre[4];
+      if (EPI == EPI_EDGEBWD) {
+#pragma unroll
+        for (int u = 0; u < 4; ++u)
+          dpre[u] = live ? __ldg(reinterpret_cast<const float4 *>(a.de + (r0 + row) * D + hf * (D / 2) + 4 * u))
+                         : make_float4(0.f, 0.f, 0.f, 0.f);
+      }
       TT_WAIT_BEGIN
       tc::mbar_wait(s.eready + (i & 3), (i >> 2) & 1);
       const int er = s.erow[(i & 3) * 128 + row];
@@ -518,15 +527,29 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
           tc::tmem_ld16(acc + c0, r);
           tc::tmem_ld_wait();
           float o[16];
-          const float *er = a.e + grow * D + cb + c0, *dr = a.de + grow * D + cb + c0;
+          float4 dcur[4];
+#pragma unroll
+          for (int u = 0; u < 4; ++u) dcur[u] = dpre[u];
+          if (c0 + 16 < DH) {
+            const float *dn = a.de + grow * D + cb + c0 + 16;
+#pragma unroll
+            for (int u = 0; u < 4; ++u)
+              dpre[u] = live ? __ldg(reinterpret_cast<const float4 *>(dn + 4 * u)) : make_float4(0.f, 0.f, 0.f, 0.f);
+          }
+          const float cexp = -aux * un * LOG2E;
 #pragma unroll
           for (int u = 0; u < 16; u += 4) {
-            float4 ev = make_float4(0.f, 0.f, 0.f, 0.f), dv = ev;
-            if (live) {
-              ev = __ldg(reinterpret_cast<const float4 *>(er + u));
-              dv = __ldg(reinterpret_cast<const float4 *>(dr + u));
+            float4 ev = make_float4(0.f, 0.f, 0.f, 0.f);
+            const float4 dv = dcur[u >> 2];
+            // e' = σ(αz) is recomputed from the accumulator exactly as EPI_EDGE formed it
+            // (same rows, weight images and MMA order -> same bits) unless a.e is given
+            if (live && a.e) ev = __ldg(reinterpret_cast<const float4 *>(a.e + grow * D + cb + c0 + u));
+            float evv[4] = {ev.x, ev.y, ev.z, ev.w};
+            const float dvv[4] = {dv.x, dv.y, dv.z, dv.w};
+            if (!a.e) {
+#pragma unroll
+              for (int t = 0; t < 4; ++t) evv[t] = fast_rcp(1.f + ex2(__uint_as_float(r[u + t]) * cexp));
             }
-            const float evv[4] = {ev.x, ev.y, ev.z, ev.w}, dvv[4] = {dv.x, dv.y, dv.z, dv.w};
 #pragma unroll
             for (int t = 0; t < 4; ++t) {
               const float z = __uint_as_float(r[u + t]) * un;
@@ -1965,7 +1988,10 @@ static int bwd_edge_impl(const occu_ctx *ctx, const DevCsr &csr, int layer, cons
   r.slope = ctx->cfg.slope;
   r.A = e_in; r.K = Ke; r.R = csr.E; r.out = DZ; r.dal = dal;
   r.wimg = tc_wimg(ctx, 1, layer); r.wfexp = tc_wfexp(ctx, 1, layer);
-  r.e = e; r.de = de; r.pin = p; r.qin = q; r.src = csr.in_src; r.dst = csr.in_dst;
+  // e' is recomputed in the epilogue (σ of the recomputed αz) when the forward formed it with
+  // the same row-GEMM (EPI_EDGE); the fused edge+gate forward stores it from another kernel
+  r.e = ctx->fuse_edge_gate ? e : nullptr;
+  r.de = de; r.pin = p; r.qin = q; r.src = csr.in_src; r.dst = csr.in_dst;
   return launch_rowgemm<D, EPI_EDGEBWD>(ctx, r, "edge_bwd_tc", st);
 }
 

@@ -214,6 +214,16 @@ class Csr:
     def on_device(self):
         return bool(self.struct.on_device)
 
+    def node_off_tensor(self, device: int = 0):
+        """Zero-copy int32 CUDA tensor view of node_off [B + 1] (device batches only)."""
+        import torch
+        s = self.struct
+        if not s.on_device:
+            raise ValueError("host batch")
+        ptr = C.cast(s.node_off, C.c_void_p).value
+        return torch.as_tensor(_DeviceArray(ptr, (s.num_graphs + 1,), "<i4"),
+                               device=torch.device("cuda", device))
+
     def arrays(self):
         """Host arrays as NumPy copies (host batches only)."""
         s = self.struct
@@ -303,8 +313,8 @@ def pack_jobs(occ, capacity=1.0):
 class _DeviceArray:
     """Zero-copy view of library-owned device memory (__cuda_array_interface__, float32)."""
 
-    def __init__(self, ptr, shape):
-        self.__cuda_array_interface__ = {"shape": tuple(shape), "typestr": "<f4",
+    def __init__(self, ptr, shape, typestr="<f4"):
+        self.__cuda_array_interface__ = {"shape": tuple(shape), "typestr": typestr,
                                          "data": (int(ptr or 0), False), "version": 3}
 
 

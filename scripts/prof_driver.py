@@ -18,6 +18,7 @@ ap.add_argument("--bf16", action="store_true")
 ap.add_argument("--graphormer", type=int, default=0)
 ap.add_argument("--decoder", action="store_true")
 ap.add_argument("--synth", action="store_true", help="inputs synthesized on the device (NEXT-4)")
+ap.add_argument("--cfg3", action="store_true", help="CFG3 (512 BERT-base / GPT-2 graphs) instead of CFG2")
 a = ap.parse_args()
 dev = torch.device("cuda", 0)
 m = occu.Model(occu.config(L=3, F_n=80, F_e=4, d=128, prec=occu.BF16 if a.bf16 else occu.FP32,
@@ -25,7 +26,7 @@ m = occu.Model(occu.config(L=3, F_n=80, F_e=4, d=128, prec=occu.BF16 if a.bf16 e
                            readout=occu.READOUT_SET_DECODER if a.decoder else occu.READOUT_MEAN))
 m.init_weights(42)
 m.set_kernel_path(a.path)
-b = configs.cfg2(a.graphs)
+b = configs.cfg3(512) if a.cfg3 else configs.cfg2(a.graphs)
 csr = m.to_device(occu.pack(b.graphs))
 nf = torch.from_numpy(b.node_feat).to(dev)
 ef = torch.from_numpy(b.edge_feat).to(dev)

@@ -138,3 +138,14 @@ def test_feature_template_hp_vector_defaults():
     assert list(templates.hp_vector("resnet50", {"batch": 20, "cin": 3})) == [20.0, 3.0, 0.0, 0.0]
     assert list(templates.hp_vector("lstm", {"batch": 128, "seq": 32})) == [128.0, 1.0, 32.0, 0.0]
     assert list(templates.hp_vector("gpt2", {"batch": 16, "cin": 3, "seq": 512})) == [16.0, 3.0, 512.0, 0.0]
+
+
+def test_mixture_arrays_match_specs():
+    from occu_gen import templates
+    specs = configs.mixture_specs(300, 1005, start=12345)
+    fam, hp = configs.mixture_arrays(300, 1005, start=12345)
+    for i, (f, h) in enumerate(specs):
+        assert configs.MIXTURE[fam[i]] == f
+        assert np.array_equal(hp[i], templates.hp_vector(f, h)), (f, h, hp[i])
+    w = configs.family_work()[fam]
+    assert np.array_equal(w, configs.spec_work(specs))
