@@ -420,6 +420,138 @@ def readout_stack(params, cfg, pk, f, hL, att_rnd=None):
     return f
 
 
+# --------------------------------------------------------------------------
+# Backward of the readout stack (NEXT-2 / NEXT-3 training; P153-P205 with Adam, P273).
+# Hand-derived, float64, in the forward's notation; every function returns the input
+# gradient(s) and adds its parameter gradients into `grads`.  Pinned by torch autograd over
+# the same forward and by central finite differences (tests/test_oracle.py).
+# --------------------------------------------------------------------------
+def _acc(grads, name, g):
+    grads[name] = grads[name] + g if name in grads else g
+
+
+def layer_norm_bwd(x, g, dy, eps=1e-5):
+    """y = x̂·g + b, x̂ = (x - μ)/sqrt(σ² + eps) per row (R33) -> (dx, dg, db)."""
+    mu = x.mean(axis=-1, keepdims=True)
+    rstd = 1.0 / np.sqrt(((x - mu) ** 2).mean(axis=-1, keepdims=True) + eps)
+    xh = (x - mu) * rstd
+    dxh = dy * g
+    dx = rstd * (dxh - dxh.mean(axis=-1, keepdims=True) - xh * (dxh * xh).mean(axis=-1, keepdims=True))
+    return dx, (dy * xh).sum(axis=0), dy.sum(axis=0)
+
+
+def ffn_bwd(x, params, p, dy, grads):
+    """FFN(x) = W2·ReLU(W1 x + b1) + b2 (R31)."""
+    a = x @ params[p + "W1"].T + params[p + "b1"]
+    t = np.maximum(a, 0.0)
+    _acc(grads, p + "W2", dy.T @ t)
+    _acc(grads, p + "b2", dy.sum(axis=0))
+    da = (dy @ params[p + "W2"]) * (a > 0)
+    _acc(grads, p + "W1", da.T @ x)
+    _acc(grads, p + "b1", da.sum(axis=0))
+    return da @ params[p + "W1"]
+
+
+def mha_bwd(X, Y, params, m, heads, dout, grads):
+    """MHA(X, Y, Y) of ``mha`` (R32) -> (dX, dY)."""
+    Q = X @ params[m + "Wq"].T + params[m + "bq"]
+    K = Y @ params[m + "Wk"].T + params[m + "bk"]
+    V = Y @ params[m + "Wv"].T + params[m + "bv"]
+    dh = Q.shape[1] // heads
+    O = np.zeros_like(Q)
+    As = []
+    for h in range(heads):
+        sl = slice(h * dh, (h + 1) * dh)
+        A = softmax_channels(Q[:, sl] @ K[:, sl].T / np.sqrt(dh))
+        O[:, sl] = A @ V[:, sl]
+        As.append(A)
+    _acc(grads, m + "Wo", dout.T @ O)
+    _acc(grads, m + "bo", dout.sum(axis=0))
+    dO = dout @ params[m + "Wo"]
+    dQ, dK, dV = np.zeros_like(Q), np.zeros_like(K), np.zeros_like(V)
+    for h in range(heads):
+        sl = slice(h * dh, (h + 1) * dh)
+        A = As[h]
+        dA = dO[:, sl] @ V[:, sl].T
+        dV[:, sl] = A.T @ dO[:, sl]
+        dS = A * (dA - np.sum(dA * A, axis=1, keepdims=True)) / np.sqrt(dh)
+        dQ[:, sl] = dS @ K[:, sl]
+        dK[:, sl] = dS.T @ Q[:, sl]
+    for w, dW, inp in (("q", dQ, X), ("k", dK, Y), ("v", dV, Y)):
+        _acc(grads, m + "W" + w, dW.T @ inp)
+        _acc(grads, m + "b" + w, dW.sum(axis=0))
+    return dQ @ params[m + "Wq"], dK @ params[m + "Wk"] + dV @ params[m + "Wv"]
+
+
+def mab_bwd(X, Y, params, m, heads, dout, grads):
+    """MAB(X, Y) = LN2(H̄ + FFN(H̄)), H̄ = LN1(X + MHA(X, Y, Y)) -> (dX, dY)."""
+    T1 = X + mha(X, Y, params, m, heads)
+    Hb = layer_norm(T1, params[m + "ln1_g"], params[m + "ln1_b"])
+    T2 = Hb + ffn(Hb, params, m + "F_")
+    dT2, dg, db = layer_norm_bwd(T2, params[m + "ln2_g"], dout)
+    _acc(grads, m + "ln2_g", dg)
+    _acc(grads, m + "ln2_b", db)
+    dHb = dT2 + ffn_bwd(Hb, params, m + "F_", dT2, grads)
+    dT1, dg, db = layer_norm_bwd(T1, params[m + "ln1_g"], dHb)
+    _acc(grads, m + "ln1_g", dg)
+    _acc(grads, m + "ln1_b", db)
+    dXa, dY = mha_bwd(X, Y, params, m, heads, dT1, grads)
+    return dT1 + dXa, dY
+
+
+def set_decoder_bwd(H, params, heads, dD, grads):
+    """Backward of ``set_decoder`` for one graph: dD [k, d] -> dH [n, d] (+ dS, parameters)."""
+    Z = ffn(H, params, "P_")
+    pma = mab(params["S"], Z, params, "M1_", heads)
+    sab = mab(pma, pma, params, "M2_", heads)
+    dsab = ffn_bwd(sab, params, "D_", dD, grads)
+    dx, dy = mab_bwd(pma, pma, params, "M2_", heads, dsab, grads)
+    dS, dZ = mab_bwd(params["S"], Z, params, "M1_", heads, dx + dy, grads)
+    _acc(grads, "S", dS)
+    return ffn_bwd(H, params, "P_", dZ, grads)
+
+
+def graphormer_layer_bwd(H, params, j, heads, dout, grads):
+    """Backward of ``graphormer_layer`` (P155, P157) for one graph: dout -> dH."""
+    g = f"G{j}_"
+    X = layer_norm(H, params[g + "ln1_g"], params[g + "ln1_b"])
+    Hb = mha(X, X, params, g, heads) + H
+    Y = layer_norm(Hb, params[g + "ln2_g"], params[g + "ln2_b"])
+    dY = ffn_bwd(Y, params, g + "F_", dout, grads)
+    dHb2, dg, db = layer_norm_bwd(Hb, params[g + "ln2_g"], dY)
+    _acc(grads, g + "ln2_g", dg)
+    _acc(grads, g + "ln2_b", db)
+    dHb = dout + dHb2
+    dXq, dXkv = mha_bwd(X, X, params, g, heads, dHb, grads)
+    dH1, dg, db = layer_norm_bwd(H, params[g + "ln1_g"], dXq + dXkv)
+    _acc(grads, g + "ln1_g", dg)
+    _acc(grads, g + "ln1_b", db)
+    return dHb + dH1
+
+
+def readout_stack_bwd(params, cfg, pk, fwd, dr, grads):
+    """dr = ∂L/∂r (the head's input) -> ∂L/∂h_L of the ANEE stack, through the decoder (or
+    the segmented mean) and the Graphormer layers in reverse, per graph."""
+    off = pk["node_off"].astype(np.int64)
+    B = pk["num_graphs"]
+    G = cfg.get("graphormer", 0)
+    hL = fwd["layers"][-1]["h"]
+    ins = [hL] + list(fwd["gph"][:-1]) if G else []
+    top = fwd["gph"][-1] if G else hL
+    if cfg.get("readout", 0) == 1:
+        dD = dr.reshape(B, cfg["k"], cfg["d"])
+        dh = np.concatenate([set_decoder_bwd(top[off[b]:off[b + 1]], params, cfg["heads"], dD[b], grads)
+                             for b in range(B)])
+    else:
+        n_b = np.diff(off)
+        gidx = pk["node_graph"].astype(np.int64)
+        dh = dr[gidx] / n_b[gidx][:, None]
+    for j in range(G - 1, -1, -1):
+        dh = np.concatenate([graphormer_layer_bwd(ins[j][off[b]:off[b + 1]], params, j, cfg["heads"],
+                                                  dh[off[b]:off[b + 1]], grads) for b in range(B)])
+    return dh
+
+
 def forward(params, cfg, pk, node_feat, edge_feat):
     """forward_anee, then (with Graphormer layers or the decoder readout) readout_stack."""
     f = forward_anee(params, cfg, pk, node_feat, edge_feat)
@@ -446,8 +578,6 @@ def mse_loss(yhat, y, global_batch=None):
 def backward(params, cfg, pk, fwd, y, global_batch=None, dsig=None):
     """dsig(layer dict) -> σ'(y) per edge and channel; default e'(1 - e') (exact
     derivative of σ at y = α z).  backward_bf16 passes e'·σ(-α z) (R28)."""
-    if cfg.get("readout", 0) == 1 or cfg.get("graphormer", 0) > 0:
-        raise NotImplementedError("training through the decoder / Graphormer layers is not built (NEXT-2/3 are inference-only)")
     slope = cfg["slope"]
     B = pk["num_graphs"]
     nb = B if global_batch is None else global_batch
@@ -462,9 +592,13 @@ def backward(params, cfg, pk, fwd, y, global_batch=None, dsig=None):
     grads["W_1"] = dc.T @ fwd["r"]
     grads["b_1"] = dc.sum(axis=0)
     dr = dc @ params["W_1"]
-    n_b = np.diff(pk["node_off"].astype(np.int64))
-    gidx = pk["node_graph"].astype(np.int64)
-    dh = dr[gidx] / n_b[gidx][:, None]
+    if cfg.get("readout", 0) == 1 or cfg.get("graphormer", 0) > 0:
+        # NEXT-2 / NEXT-3: through the decoder readout and the Graphormer layers
+        dh = readout_stack_bwd(params, cfg, pk, fwd, dr, grads)
+    else:
+        n_b = np.diff(pk["node_off"].astype(np.int64))
+        gidx = pk["node_graph"].astype(np.int64)
+        dh = dr[gidx] / n_b[gidx][:, None]
     de_out = None
     deg = np.diff(pk["in_ptr"].astype(np.int64))
     for i in range(cfg["L"] - 1, -1, -1):

@@ -874,3 +874,99 @@ def test_mha_fp16_rounded_variant_limits():
     r16 = oracle.mha(X, X, p, "G_", heads, rnd=oracle.fp16_round)
     assert np.linalg.norm(r16 - ref) <= 4e-3 * np.linalg.norm(ref)
     assert not np.array_equal(r16, ref)
+
+
+# ------------------------------------------ NEXT-2 / NEXT-3 training: readout-stack backward
+def torch_full_loss(p, c, pk, X, EF, y, gb=None):
+    """Independent forward of the paper's full model (ANEE -> Graphormer layers -> decoder or
+    mean -> head, MSE) built from torch.nn.functional (layer_norm, multi_head_attention_forward,
+    linear), differentiated by autograd in float64."""
+    torch = pytest.importorskip("torch")
+    F = torch.nn.functional
+    T = {k: torch.tensor(v, dtype=torch.float64, requires_grad=True) for k, v in p.items()}
+    s = torch.tensor(pk["in_src"].astype(np.int64))
+    t = torch.tensor(pk["in_dst"].astype(np.int64))
+    h = torch.tensor(X, dtype=torch.float64)
+    e = torch.tensor(EF, dtype=torch.float64)[torch.tensor(pk["in_eid"].astype(np.int64))]
+    lrelu = lambda x: F.leaky_relu(x, c["slope"])
+    N, d, heads = pk["num_nodes"], c["d"], c["heads"]
+    for i in range(c["L"]):
+        hb = lrelu(h @ T[f"W_u{i}"].T)
+        al = hb[s] @ T[f"a_s{i}"] + hb[t] @ T[f"a_d{i}"]
+        e = torch.sigmoid(al[:, None] * (e @ T[f"W_e{i}"].T))
+        g = torch.softmax(e @ T[f"W_m{i}"].T, dim=1)
+        h = lrelu(torch.zeros(N, d, dtype=torch.float64).index_add(0, t, g * hb[s]))
+
+    def ffn(x, q):
+        return F.linear(F.relu(F.linear(x, T[q + "W1"], T[q + "b1"])), T[q + "W2"], T[q + "b2"])
+
+    def att(Xq, Y, m):
+        o, _ = F.multi_head_attention_forward(
+            Xq[:, None], Y[:, None], Y[:, None], d, heads,
+            torch.cat([T[m + "Wq"], T[m + "Wk"], T[m + "Wv"]]),
+            torch.cat([T[m + "bq"], T[m + "bk"], T[m + "bv"]]), None, None, False, 0.0,
+            T[m + "Wo"], T[m + "bo"], training=False, need_weights=False)
+        return o[:, 0]
+
+    def ln(x, q):
+        return F.layer_norm(x, (d,), T[q + "_g"], T[q + "_b"], 1e-5)
+
+    def mab(Xq, Y, m):
+        Hb = ln(Xq + att(Xq, Y, m), m + "ln1")
+        return ln(Hb + ffn(Hb, m + "F_"), m + "ln2")
+
+    off = pk["node_off"].astype(np.int64)
+    rows = []
+    for b in range(pk["num_graphs"]):
+        H = h[off[b]:off[b + 1]]
+        for j in range(c["graphormer"]):
+            g_ = f"G{j}_"
+            Hb = att(ln(H, g_ + "ln1"), ln(H, g_ + "ln1"), g_) + H
+            H = ffn(ln(Hb, g_ + "ln2"), g_ + "F_") + Hb
+        if c["readout"] == 1:
+            pma = mab(T["S"], ffn(H, "P_"), "M1_")
+            rows.append(ffn(mab(pma, pma, "M2_"), "D_").reshape(-1))
+        else:
+            rows.append(H.mean(dim=0))
+    r = torch.stack(rows)
+    yh = lrelu(r @ T["W_1"].T + T["b_1"]) @ T["w_2"] + T["b_2"][0]
+    nb = len(y) if gb is None else gb
+    loss = ((yh - torch.tensor(y, dtype=torch.float64)) ** 2).sum() / nb
+    loss.backward()
+    return float(loss), {k: v.grad.numpy() for k, v in T.items()}
+
+
+def _stack_params(c, seed):
+    p = gph_params(c, seed)
+    rng = np.random.default_rng(seed + 100)
+    if c["readout"] == 1:
+        for m in ("M1_", "M2_"):
+            for ln_ in ("ln1", "ln2"):
+                p[m + ln_ + "_g"] = 1.0 + 0.3 * rng.standard_normal(c["d"])
+                p[m + ln_ + "_b"] = 0.2 * rng.standard_normal(c["d"])
+    return p
+
+
+@pytest.mark.parametrize("G,heads,readout", [(2, 4, 0), (0, 2, 1), (2, 4, 1), (1, 1, 1)])
+def test_readout_stack_backward_matches_torch_autograd(G, heads, readout):
+    c = gph_cfg(G=G, heads=heads, readout=readout, k=3)
+    b = configs.random_dag_batch(4, 900 + G + heads + readout, max_nodes=16, hub=True)
+    p = _stack_params(c, 21 + G)
+    pk = oracle.pack(b.graphs)
+    loss, grads = oracle.backward(p, c, pk, oracle.forward(p, c, pk, b.node_feat, b.edge_feat),
+                                  b.targets, global_batch=7)
+    tl, tg = torch_full_loss(p, c, pk, b.node_feat, b.edge_feat, b.targets, gb=7)
+    assert abs(loss - tl) <= 1e-12 * abs(tl)
+    assert set(grads) == set(p)
+    for k in p:
+        assert np.allclose(grads[k], tg[k], rtol=1e-8, atol=1e-13 * max(1, np.abs(tg[k]).max())), k
+
+
+@pytest.mark.parametrize("G,readout", [(1, 1), (2, 0)])
+def test_readout_stack_backward_finite_differences(G, readout):
+    """Central differences through the whole stack on a tiny model (d = 4, 2 heads, k = 2)."""
+    c = gph_cfg(G=G, heads=2, d=4, L=1, readout=readout, k=2)
+    c["F_n"], c["F_e"] = 5, 3
+    b = configs.random_dag_batch(3, 70 + G, max_nodes=6, f_n=5, f_e=3, hub=True)
+    p = _stack_params(c, 31 + G)
+    fd_check(c, b, p, tol=2e-6)
