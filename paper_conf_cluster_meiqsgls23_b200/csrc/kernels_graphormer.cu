@@ -816,7 +816,8 @@ int ln_launch(const occu_ctx *ctx, const float *X, int N, const float *g, const 
 }  // namespace
 
 int launch_graphormer_layer(const occu_ctx *ctx, const DevCsr &csr, int j, const float *h_in,
-                            float *h_out, float *X, float *QKV, float *O, cudaStream_t st) {
+                            float *h_out, float *X, float *QKV, float *O, cudaStream_t st,
+                            const GphSave *sv) {
   const occu_config &cf = ctx->cfg;
   const GphOff &G = ctx->layout.G[j];
   const float *P = ctx->params.as<float>();
@@ -824,6 +825,11 @@ int launch_graphormer_layer(const occu_ctx *ctx, const DevCsr &csr, int j, const
   if (N <= 0) return 0;
   const size_t ND = size_t(N) * D;
   float *Qb = QKV, *Kb = QKV + ND, *Vb = QKV + 2 * ND;
+  float *X2 = X, *Hb = Kb, *T = Qb;        // inference: scratch reused stage by stage
+  if (sv) {                                 // training: every intermediate kept (backward)
+    X = sv->X1; Qb = sv->Q; Kb = sv->K; Vb = sv->V; O = sv->O;
+    Hb = sv->Hb; X2 = sv->X2; T = sv->T;
+  }
   int n = 0, r;
   auto ln = [&](const float *x, size_t g, size_t b, float *y) {
     return D == 64 ? ln_launch<64>(ctx, x, N, P + g, P + b, y, st)
@@ -887,13 +893,13 @@ int launch_graphormer_layer(const occu_ctx *ctx, const DevCsr &csr, int j, const
   }
   OCCU_PROF_END(ctx);
   ++n;
-  float *Hb = Kb;          // K is dead after the attention: h̄ lives there
+  // h̄ (inference: K is dead after the attention, h̄ lives there)
   if ((r = launch_bias_add_tc(ctx, O, D, N, 3, slot, P + G.bo, h_in, Hb, "gph_out_tc", st)) < 0) return r;
   n += r;
   // h' = FFN(LN(h̄)) + h̄
-  n += ln(Hb, G.ln2_g, G.ln2_b, X);
-  float *T = Qb;           // FFN hidden rows
-  if ((r = launch_bias_tc(ctx, X, D, N, 4, slot, P + G.F.b1, true, T, "gph_ffn_tc", st)) < 0) return r;
+  n += ln(Hb, G.ln2_g, G.ln2_b, X2);
+  // FFN hidden rows (inference: in Q's place)
+  if ((r = launch_bias_tc(ctx, X2, D, N, 4, slot, P + G.F.b1, true, T, "gph_ffn_tc", st)) < 0) return r;
   n += r;
   if ((r = launch_bias_add_tc(ctx, T, D, N, 5, slot, P + G.F.b2, Hb, h_out, "gph_ffn_tc", st)) < 0) return r;
   n += r;

@@ -1938,7 +1938,9 @@ int launch_head_backward(occu_ctx *ctx, const DevCsr &csr, const float *targets,
   OCCU_PROF_END(ctx);
   LAUNCH_CHECK();
   OCCU_PROF_BEGIN(ctx, "broadcast_dh", st);
-  const bool tcb = ctx->path != 1 && tc_supported(cf);    // TC backward consumes dA directly
+  // TC backward consumes dA directly; with Graphormer layers dr/n_b is the gradient of the
+  // stack's top states and the mask is applied below the stack (launch_mask_dA)
+  const bool tcb = ctx->path != 1 && tc_supported(cf) && cf.graphormer == 0;
   broadcast_dh_kernel<<<grid_for(long(csr.N) * cf.d / 4, 256, 16 * ctx->num_sms), 256, 0, st>>>(
       w.dr.as<float>(), csr.node_graph, csr.node_off, csr.N, cf.d,
       tcb ? w.h[cf.L - 1].ptr : nullptr, cf.prec == OCCU_BF16 ? 1 : 0, csr.in_ptr,

@@ -1,0 +1,461 @@
+// Training through the paper's readout stack (P153-P205 with
+// Adam, P273): the backward of the Graphormer layers (pre-LN MHA + FFN over each graph's node
+// set, R35-R37) and the building blocks the decoder backward shares with them.
+//
+//   Graphormer layer (forward, kernels_graphormer.cu):  X1 = LN1(H), Q|K|V = X1 W_{q,k,v}ᵀ + b,
+//     O = softmax(Q Kᵀ/√d_h) V per graph and head, h̄ = O W_oᵀ + b_o + H, X2 = LN2(h̄),
+//     T = ReLU(X2 W1ᵀ + b1), out = T W2ᵀ + b2 + h̄.
+//   Backward (this file), with dX = dY·W row-GEMMs on tensor cores against transposed fp16x2
+//   weight images (gph_tslot), weight gradients XᵀY on the split-K tensor-core wgrad kernel,
+//   bias / LayerNorm parameter gradients as fixed-order column sums (float64 partials):
+//     dT = (dout W2) ⊙ [T > 0]; dX2 = dT W1; dh̄ = dout + LN2ᵀ(dX2); dO = dh̄ W_o;
+//     attention backward per graph and head (below); dX1 = dQ W_q + dK W_k + dV W_v;
+//     dH = dh̄ + LN1ᵀ(dX1).
+//   Attention backward (FP32 CUDA cores, two passes, no atomics): stats m_i, l_i of every
+//   query row over its own graph's keys and D_i = <dO_i, O_i>; then
+//     dQ_i = Σ_j P_ij (dO_i·V_j − D_i) K_j / √d_h        (thread = query row)
+//     dV_j = Σ_i P_ij dO_i,  dK_j = Σ_i P_ij (dO_i·V_j − D_i) Q_i / √d_h   (thread = key row)
+//   with P_ij = exp(s_ij − m_i)/l_i recomputed, keys / queries of the block's graphs staged
+//   through shared memory; sums in ascending index order (deterministic).
+#include <cuda_runtime.h>
+#include <math.h>
+#include <stdint.h>
+
+#include <algorithm>
+
+#include "occu_internal.h"
+
+namespace occu {
+namespace {
+
+constexpr int ST = 256;          // threads per block (row kernels)
+
+#define SK_CHECK()                                  \
+  do {                                              \
+    cudaError_t e__ = cudaGetLastError();           \
+    if (e__ != cudaSuccess) return -int(e__);       \
+  } while (0)
+
+int grid_rows(long rows, int rows_per_block, int cap) {
+  return int(std::max<long>(1, std::min<long>((rows + rows_per_block - 1) / rows_per_block, cap)));
+}
+
+// ---------------------------------------------------------------------------------------
+// LayerNorm backward (R33), warp per row, V = D/32 channels per lane (lane-contiguous):
+//   x̂ = (x − μ)·rstd,  dx = add + rstd·(g⊙dy − mean(g⊙dy) − x̂·mean(g⊙dy⊙x̂)),
+// and per-block partial column sums of dy⊙x̂ (dγ) and dy (dβ) in float64.
+template <int D>
+__global__ void __launch_bounds__(ST) ln_bwd_kernel(const float *__restrict__ x, const float *__restrict__ gam,
+                                                    const float *__restrict__ dy, const float *__restrict__ add,
+                                                    float *__restrict__ dx, long R, double *__restrict__ part) {
+  constexpr int V = D / 32;
+  const int lane = threadIdx.x & 31, wl = threadIdx.x >> 5;
+  double pg[V], pb[V];
+  float gv[V];
+#pragma unroll
+  for (int c = 0; c < V; ++c) {
+    pg[c] = pb[c] = 0.0;
+    gv[c] = __ldg(gam + lane * V + c);
+  }
+  const long nw = long(gridDim.x) * (ST / 32);
+  for (long r = long(blockIdx.x) * (ST / 32) + wl; r < R; r += nw) {
+    float xv[V], dv[V];
+#pragma unroll
+    for (int c = 0; c < V; ++c) {
+      xv[c] = __ldg(x + r * D + lane * V + c);
+      dv[c] = __ldg(dy + r * D + lane * V + c);
+    }
+    float s = 0.f;
+#pragma unroll
+    for (int c = 0; c < V; ++c) s += xv[c];
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+    const float mu = s * (1.f / float(D));
+    float q = 0.f;
+#pragma unroll
+    for (int c = 0; c < V; ++c) q = fmaf(xv[c] - mu, xv[c] - mu, q);
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) q += __shfl_xor_sync(0xffffffffu, q, o);
+    const float rstd = rsqrtf(q * (1.f / float(D)) + 1e-5f);
+    float a1 = 0.f, a2 = 0.f, xh[V], gd[V];
+#pragma unroll
+    for (int c = 0; c < V; ++c) {
+      xh[c] = (xv[c] - mu) * rstd;
+      gd[c] = gv[c] * dv[c];
+      a1 += gd[c];
+      a2 = fmaf(gd[c], xh[c], a2);
+      pg[c] = fma(double(dv[c]), double(xh[c]), pg[c]);
+      pb[c] += double(dv[c]);
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+      a1 += __shfl_xor_sync(0xffffffffu, a1, o);
+      a2 += __shfl_xor_sync(0xffffffffu, a2, o);
+    }
+    a1 *= 1.f / float(D);
+    a2 *= 1.f / float(D);
+#pragma unroll
+    for (int c = 0; c < V; ++c) {
+      float o = rstd * (gd[c] - a1 - xh[c] * a2);
+      if (add) o += __ldg(add + r * D + lane * V + c);
+      dx[r * D + lane * V + c] = o;
+    }
+  }
+  __shared__ double red[ST / 32][2 * D];
+#pragma unroll
+  for (int c = 0; c < V; ++c) {
+    red[wl][lane * V + c] = pg[c];
+    red[wl][D + lane * V + c] = pb[c];
+  }
+  __syncthreads();
+  for (int o = threadIdx.x; o < 2 * D; o += ST) {
+    double t = 0.0;
+    for (int w = 0; w < ST / 32; ++w) t += red[w][o];
+    part[long(blockIdx.x) * 2 * D + o] = t;
+  }
+}
+
+// Per-block partial column sums of X [R][D] (bias gradients), float64, warp per row.
+template <int D>
+__global__ void __launch_bounds__(ST) colsum_kernel(const float *__restrict__ X, long R,
+                                                    double *__restrict__ part) {
+  constexpr int V = D / 32;
+  const int lane = threadIdx.x & 31, wl = threadIdx.x >> 5;
+  double acc[V];
+#pragma unroll
+  for (int c = 0; c < V; ++c) acc[c] = 0.0;
+  const long nw = long(gridDim.x) * (ST / 32);
+  for (long r = long(blockIdx.x) * (ST / 32) + wl; r < R; r += nw) {
+#pragma unroll
+    for (int c = 0; c < V; ++c) acc[c] += double(__ldg(X + r * D + lane * V + c));
+  }
+  __shared__ double red[ST / 32][D];
+#pragma unroll
+  for (int c = 0; c < V; ++c) red[wl][lane * V + c] = acc[c];
+  __syncthreads();
+  for (int o = threadIdx.x; o < D; o += ST) {
+    double t = 0.0;
+    for (int w = 0; w < ST / 32; ++w) t += red[w][o];
+    part[long(blockIdx.x) * D + o] = t;
+  }
+}
+
+// out[c] = Σ_b part[b][c] in block order (float64), c < C.  out2 (nullable) takes columns
+// [C, 2C) of a [nblk][2C] partial array.
+__global__ void col_reduce_kernel(const double *__restrict__ part, int nblk, int C, int ld,
+                                  float *__restrict__ out, float *__restrict__ out2) {
+  const int c = blockIdx.x * blockDim.x + threadIdx.x;
+  if (c >= C) return;
+  double a = 0.0, b = 0.0;
+  for (int k = 0; k < nblk; ++k) {
+    a += part[long(k) * ld + c];
+    if (out2) b += part[long(k) * ld + C + c];
+  }
+  out[c] = float(a);
+  if (out2) out2[c] = float(b);
+}
+
+// dA = dh ⊙ LReLU'(h) (÷ deg for MEAN) — sign(A) = sign(h) (R7).
+__global__ void mask_dA_kernel(const float *__restrict__ dh, const float *__restrict__ h,
+                               const int32_t *__restrict__ in_ptr, long N, int D, int mean,
+                               float slope, float *__restrict__ dA) {
+  const long total = N * D / 4;
+  for (long i = blockIdx.x * long(blockDim.x) + threadIdx.x; i < total; i += long(gridDim.x) * blockDim.x) {
+    const long u = i / (D / 4);
+    const float4 g = __ldg(reinterpret_cast<const float4 *>(dh) + i);
+    const float4 x = __ldg(reinterpret_cast<const float4 *>(h) + i);
+    float dsc = 1.f;
+    if (mean) {
+      const int deg = __ldg(in_ptr + u + 1) - __ldg(in_ptr + u);
+      dsc = float(deg > 0 ? deg : 1);
+    }
+    float4 o;
+    o.x = g.x * (x.x > 0.f ? 1.f : slope) / dsc;
+    o.y = g.y * (x.y > 0.f ? 1.f : slope) / dsc;
+    o.z = g.z * (x.z > 0.f ? 1.f : slope) / dsc;
+    o.w = g.w * (x.w > 0.f ? 1.f : slope) / dsc;
+    reinterpret_cast<float4 *>(dA)[i] = o;
+  }
+}
+
+// ---------------------------------------------------------------------------------------
+// Attention backward (per graph, per head; block-diagonal over the batch).
+struct AttnBwdArgs {
+  const float *Q, *K, *V, *O, *dO;   // [N][D]
+  const int32_t *node_off, *node_graph;
+  float *dQ, *dK, *dV;               // [N][D]
+  float *stats;                      // [N][heads][3]: m, l, D
+  int N, D, heads;
+  float scale;                       // 1 / sqrt(d_h)
+};
+
+constexpr int ABT = 128;             // rows per block
+constexpr int TK = 32;               // staged rows per tile
+
+// Pass 1 + dQ: thread = query row i of head blockIdx.y.
+template <int DH>
+__global__ void __launch_bounds__(ABT) attn_bwd_q_kernel(const AttnBwdArgs a) {
+  __shared__ float sk[TK][DH], sv[TK][DH];
+  const int h = blockIdx.y;
+  const long i0 = long(blockIdx.x) * ABT;
+  const long i = i0 + threadIdx.x;
+  const bool live = i < a.N;
+  const long il = min(i0 + ABT, long(a.N)) - 1;
+  const int b0 = __ldg(a.node_graph + i0), b1 = __ldg(a.node_graph + il);
+  const int ub = __ldg(a.node_off + b0), ue = __ldg(a.node_off + b1 + 1);   // union key range
+  int kb = 0, ke = 0;
+  float q[DH], go[DH], acc[DH];
+  float Di = 0.f;
+  if (live) {
+    const int b = __ldg(a.node_graph + i);
+    kb = __ldg(a.node_off + b);
+    ke = __ldg(a.node_off + b + 1);
+#pragma unroll
+    for (int c = 0; c < DH; ++c) {
+      q[c] = __ldg(a.Q + i * a.D + h * DH + c) * a.scale;
+      go[c] = __ldg(a.dO + i * a.D + h * DH + c);
+      Di = fmaf(go[c], __ldg(a.O + i * a.D + h * DH + c), Di);
+      acc[c] = 0.f;
+    }
+  }
+  // pass 1: row maximum and normaliser over the own graph's keys
+  float m = -INFINITY, l = 0.f;
+  for (int t0 = ub; t0 < ue; t0 += TK) {
+    __syncthreads();
+    for (int e = threadIdx.x; e < TK * DH; e += ABT) {
+      const int rr = e / DH, cc = e % DH;
+      sk[rr][cc] = t0 + rr < ue ? __ldg(a.K + long(t0 + rr) * a.D + h * DH + cc) : 0.f;
+    }
+    __syncthreads();
+    if (live) {
+      const int jb = max(kb, t0), je = min(ke, t0 + TK);
+      for (int j = jb; j < je; ++j) {
+        float s = 0.f;
+#pragma unroll
+        for (int c = 0; c < DH; ++c) s = fmaf(q[c], sk[j - t0][c], s);
+        if (s > m) {
+          l = l * expf(m - s) + 1.f;
+          m = s;
+        } else {
+          l += expf(s - m);
+        }
+      }
+    }
+  }
+  const float inv_l = 1.f / l;
+  // pass 2: dQ
+  for (int t0 = ub; t0 < ue; t0 += TK) {
+    __syncthreads();
+    for (int e = threadIdx.x; e < TK * DH; e += ABT) {
+      const int rr = e / DH, cc = e % DH;
+      const bool in = t0 + rr < ue;
+      sk[rr][cc] = in ? __ldg(a.K + long(t0 + rr) * a.D + h * DH + cc) : 0.f;
+      sv[rr][cc] = in ? __ldg(a.V + long(t0 + rr) * a.D + h * DH + cc) : 0.f;
+    }
+    __syncthreads();
+    if (live) {
+      const int jb = max(kb, t0), je = min(ke, t0 + TK);
+      for (int j = jb; j < je; ++j) {
+        float s = 0.f, dp = 0.f;
+#pragma unroll
+        for (int c = 0; c < DH; ++c) {
+          s = fmaf(q[c], sk[j - t0][c], s);
+          dp = fmaf(go[c], sv[j - t0][c], dp);
+        }
+        const float p = expf(s - m) * inv_l;
+        const float ds = p * (dp - Di);
+#pragma unroll
+        for (int c = 0; c < DH; ++c) acc[c] = fmaf(ds, sk[j - t0][c], acc[c]);
+      }
+    }
+  }
+  if (live) {
+#pragma unroll
+    for (int c = 0; c < DH; ++c) a.dQ[i * a.D + h * DH + c] = acc[c] * a.scale;
+    float *stt = a.stats + (i * a.heads + h) * 3;
+    stt[0] = m;
+    stt[1] = l;
+    stt[2] = Di;
+  }
+}
+
+// dK, dV: thread = key row j of head blockIdx.y; queries of the block's graphs staged.
+template <int DH>
+__global__ void __launch_bounds__(ABT) attn_bwd_kv_kernel(const AttnBwdArgs a) {
+  __shared__ float sq[TK][DH], sg[TK][DH], ss[TK][3];
+  const int h = blockIdx.y;
+  const long j0 = long(blockIdx.x) * ABT;
+  const long j = j0 + threadIdx.x;
+  const bool live = j < a.N;
+  const long jl = min(j0 + ABT, long(a.N)) - 1;
+  const int b0 = __ldg(a.node_graph + j0), b1 = __ldg(a.node_graph + jl);
+  const int ub = __ldg(a.node_off + b0), ue = __ldg(a.node_off + b1 + 1);
+  int qb = 0, qe = 0;
+  float k[DH], v[DH], dk[DH], dv[DH];
+  if (live) {
+    const int b = __ldg(a.node_graph + j);
+    qb = __ldg(a.node_off + b);
+    qe = __ldg(a.node_off + b + 1);
+#pragma unroll
+    for (int c = 0; c < DH; ++c) {
+      k[c] = __ldg(a.K + j * a.D + h * DH + c);
+      v[c] = __ldg(a.V + j * a.D + h * DH + c);
+      dk[c] = dv[c] = 0.f;
+    }
+  }
+  for (int t0 = ub; t0 < ue; t0 += TK) {
+    __syncthreads();
+    for (int e = threadIdx.x; e < TK * DH; e += ABT) {
+      const int rr = e / DH, cc = e % DH;
+      const bool in = t0 + rr < ue;
+      sq[rr][cc] = in ? __ldg(a.Q + long(t0 + rr) * a.D + h * DH + cc) * a.scale : 0.f;
+      sg[rr][cc] = in ? __ldg(a.dO + long(t0 + rr) * a.D + h * DH + cc) : 0.f;
+    }
+    for (int e = threadIdx.x; e < TK * 3; e += ABT) {
+      const int rr = e / 3, cc = e % 3;
+      ss[rr][cc] = t0 + rr < ue ? a.stats[(long(t0 + rr) * a.heads + h) * 3 + cc] : 1.f;
+    }
+    __syncthreads();
+    if (live) {
+      const int ib = max(qb, t0), ie = min(qe, t0 + TK);
+      for (int i = ib; i < ie; ++i) {
+        const int r = i - t0;
+        float s = 0.f, dp = 0.f;
+#pragma unroll
+        for (int c = 0; c < DH; ++c) {
+          s = fmaf(sq[r][c], k[c], s);
+          dp = fmaf(sg[r][c], v[c], dp);
+        }
+        const float p = expf(s - ss[r][0]) / ss[r][1];
+        const float ds = p * (dp - ss[r][2]);
+#pragma unroll
+        for (int c = 0; c < DH; ++c) {
+          dv[c] = fmaf(p, sg[r][c], dv[c]);
+          dk[c] = fmaf(ds, sq[r][c], dk[c]);      // sq already carries 1/√d_h
+        }
+      }
+    }
+  }
+  if (live) {
+#pragma unroll
+    for (int c = 0; c < DH; ++c) {
+      a.dK[j * a.D + h * DH + c] = dk[c];
+      a.dV[j * a.D + h * DH + c] = dv[c];
+    }
+  }
+}
+
+}  // namespace
+
+// ---- launchers ---------------------------------------------------------------------------
+// bias-style gradient: out[c] = Σ_r X[r][c] (fixed order)
+static int colsum(occu_ctx *ctx, const float *X, long R, float *out, cudaStream_t st) {
+  const int D = ctx->cfg.d;
+  const int nb = grid_rows(R, ST / 32 * 8, 4 * ctx->num_sms);
+  if (ctx->ws.dpart.ensure(size_t(nb) * 2 * D * 8) != cudaSuccess) return -int(cudaErrorMemoryAllocation);
+  double *part = reinterpret_cast<double *>(ctx->ws.dpart.ptr);
+  OCCU_PROF_BEGIN(ctx, "stack_colsum", st);
+  if (D == 64) colsum_kernel<64><<<nb, ST, 0, st>>>(X, R, part);
+  else colsum_kernel<128><<<nb, ST, 0, st>>>(X, R, part);
+  col_reduce_kernel<<<(D + 127) / 128, 128, 0, st>>>(part, nb, D, D, out, nullptr);
+  OCCU_PROF_END(ctx);
+  SK_CHECK();
+  return 2;
+}
+
+// dx = add + LNᵀ(dy) for x = LN input; dγ, dβ into gg, gb.
+static int ln_bwd(occu_ctx *ctx, const float *x, const float *gam, const float *dy, const float *add,
+                  float *dx, long R, float *gg, float *gb, cudaStream_t st) {
+  const int D = ctx->cfg.d;
+  const int nb = grid_rows(R, ST / 32 * 8, 4 * ctx->num_sms);
+  if (ctx->ws.dpart.ensure(size_t(nb) * 2 * D * 8) != cudaSuccess) return -int(cudaErrorMemoryAllocation);
+  double *part = reinterpret_cast<double *>(ctx->ws.dpart.ptr);
+  OCCU_PROF_BEGIN(ctx, "stack_ln_bwd", st);
+  if (D == 64) ln_bwd_kernel<64><<<nb, ST, 0, st>>>(x, gam, dy, add, dx, R, part);
+  else ln_bwd_kernel<128><<<nb, ST, 0, st>>>(x, gam, dy, add, dx, R, part);
+  col_reduce_kernel<<<(D + 127) / 128, 128, 0, st>>>(part, nb, D, 2 * D, gg, gb);
+  OCCU_PROF_END(ctx);
+  SK_CHECK();
+  return 2;
+}
+
+int launch_mask_dA(const occu_ctx *ctx, const DevCsr &csr, const float *dh, const float *h, float *dA,
+                   cudaStream_t st) {
+  const occu_config &c = ctx->cfg;
+  const long n4 = long(csr.N) * c.d / 4;
+  OCCU_PROF_BEGIN(ctx, "stack_mask_dA", st);
+  mask_dA_kernel<<<grid_rows(n4, 256, 16 * ctx->num_sms), 256, 0, st>>>(
+      dh, h, csr.in_ptr, csr.N, c.d, c.aggr == OCCU_AGGR_MEAN, c.slope, dA);
+  OCCU_PROF_END(ctx);
+  SK_CHECK();
+  return 1;
+}
+
+int launch_graphormer_layer_bwd(occu_ctx *ctx, const DevCsr &csr, int j, const float *h_in,
+                                const GphSave &sv, const float *dout, float *dh_in, float *scratch,
+                                cudaStream_t st) {
+  const occu_config &cf = ctx->cfg;
+  const GphOff &G = ctx->layout.G[j];
+  const float *P = ctx->params.as<float>();
+  float *Gr = ctx->grads.as<float>();
+  const int D = cf.d, N = csr.N, ts = gph_tslot(cf, j);
+  if (N <= 0) return 0;
+  const size_t ND = size_t(N) * D;
+  float *s1 = scratch, *s2 = scratch + ND, *s3 = scratch + 2 * ND, *s4 = scratch + 3 * ND,
+        *s5 = scratch + 4 * ND;
+  float *stats = scratch + 5 * ND;                        // [N][heads][3]
+  int n = 0, r;
+#define SKR(call)                  \
+  do {                             \
+    if ((r = (call)) < 0) return r; \
+    n += r;                        \
+  } while (0)
+  // FFN: dT = (dout W2) ⊙ [T > 0]; dW2 = doutᵀ T; db2; dX2 = dT W1; dW1 = dTᵀ X2; db1
+  SKR(launch_plain_masked_tc(ctx, dout, D, N, 5, ts, nullptr, s1, "stack_gemm_tc", st, sv.T, 0.f));
+  SKR(launch_wgrad(ctx, dout, D, sv.T, D, N, Gr + G.F.W2, st, false));
+  SKR(colsum(ctx, dout, N, Gr + G.F.b2, st));
+  SKR(launch_plain_tc(ctx, s1, D, N, 4, ts, nullptr, s2, "stack_gemm_tc", st));
+  SKR(launch_wgrad(ctx, s1, D, sv.X2, D, N, Gr + G.F.W1, st, false));
+  SKR(colsum(ctx, s1, N, Gr + G.F.b1, st));
+  // dh̄ = dout + LN2ᵀ(dX2)
+  SKR(ln_bwd(ctx, sv.Hb, P + G.ln2_g, s2, dout, s3, N, Gr + G.ln2_g, Gr + G.ln2_b, st));
+  // dO = dh̄ W_o; dW_o = dh̄ᵀ O; db_o
+  SKR(launch_plain_tc(ctx, s3, D, N, 3, ts, nullptr, s2, "stack_gemm_tc", st));
+  SKR(launch_wgrad(ctx, s3, D, sv.O, D, N, Gr + G.Wo, st, false));
+  SKR(colsum(ctx, s3, N, Gr + G.bo, st));
+  // attention backward: dQ -> s1, dK -> s4, dV -> s5
+  AttnBwdArgs a;
+  a.Q = sv.Q; a.K = sv.K; a.V = sv.V; a.O = sv.O; a.dO = s2;
+  a.node_off = csr.node_off; a.node_graph = csr.node_graph;
+  a.dQ = s1; a.dK = s4; a.dV = s5; a.stats = stats;
+  a.N = N; a.D = D; a.heads = cf.heads;
+  const int dh = D / cf.heads;
+  a.scale = 1.f / sqrtf(float(dh));
+  const dim3 grid((N + ABT - 1) / ABT, cf.heads);
+  OCCU_PROF_BEGIN(ctx, "stack_attn_bwd", st);
+  switch (dh) {
+    case 16: attn_bwd_q_kernel<16><<<grid, ABT, 0, st>>>(a); attn_bwd_kv_kernel<16><<<grid, ABT, 0, st>>>(a); break;
+    case 32: attn_bwd_q_kernel<32><<<grid, ABT, 0, st>>>(a); attn_bwd_kv_kernel<32><<<grid, ABT, 0, st>>>(a); break;
+    case 64: attn_bwd_q_kernel<64><<<grid, ABT, 0, st>>>(a); attn_bwd_kv_kernel<64><<<grid, ABT, 0, st>>>(a); break;
+    default: return -int(cudaErrorInvalidValue);
+  }
+  OCCU_PROF_END(ctx);
+  SK_CHECK();
+  n += 2;
+  // projections: dW_{q,k,v} = d{Q,K,V}ᵀ X1, biases; dX1 = dQ W_q + dK W_k + dV W_v -> s2
+  SKR(launch_wgrad(ctx, s1, D, sv.X1, D, N, Gr + G.Wq, st, false));
+  SKR(colsum(ctx, s1, N, Gr + G.bq, st));
+  SKR(launch_wgrad(ctx, s4, D, sv.X1, D, N, Gr + G.Wk, st, false));
+  SKR(colsum(ctx, s4, N, Gr + G.bk, st));
+  SKR(launch_wgrad(ctx, s5, D, sv.X1, D, N, Gr + G.Wv, st, false));
+  SKR(colsum(ctx, s5, N, Gr + G.bv, st));
+  SKR(launch_plain_tc(ctx, s1, D, N, 0, ts, nullptr, s2, "stack_gemm_tc", st));
+  SKR(launch_plain_tc(ctx, s4, D, N, 1, ts, s2, s2, "stack_gemm_tc", st));
+  SKR(launch_plain_tc(ctx, s5, D, N, 2, ts, s2, s2, "stack_gemm_tc", st));
+  // dH = dh̄ + LN1ᵀ(dX1)
+  SKR(ln_bwd(ctx, h_in, P + G.ln1_g, s2, s3, dh_in, N, Gr + G.ln1_g, Gr + G.ln1_b, st));
+#undef SKR
+  return n;
+}
+
+}  // namespace occu

@@ -1726,7 +1726,8 @@ int tc_prepare_weights(occu_ctx *ctx, cudaStream_t st) {
   const ParamLayout &L = ctx->layout;
   // slots: 6 kinds per ANEE layer, plus "layer" L for the decoder's FFN (kinds 0, 1) and
   // "layer" L + 1 + j for Graphormer layer j (kinds 0-5: W_q, W_k, W_v, W_o, FFN W1, W2)
-  const size_t nslot = size_t(c.L + 1 + c.graphormer) * 6;
+  // + "layer" L + 1 + G + j: Graphormer layer j's transposed matrices (backward, gph_tslot)
+  const size_t nslot = size_t(c.L + 1 + 2 * c.graphormer) * 6;
   if (ctx->wimg.ensure(nslot * WIMG_MAX) != cudaSuccess ||
       ctx->wfexp.ensure(nslot * 2 * sizeof(int)) != cudaSuccess ||
       ctx->wjobs.ensure(nslot * sizeof(WImageJob)) != cudaSuccess)
@@ -1773,6 +1774,10 @@ int tc_prepare_weights(occu_ctx *ctx, cudaStream_t st) {
       jb.img = const_cast<uint8_t *>(tc_wimg(ctx, kind, c.L + 1 + j));
       jb.fexp = const_cast<int *>(tc_wfexp(ctx, kind, c.L + 1 + j));
       jobs.push_back(jb);
+      jb.transW = 1;                   // dX = dY·W of the backward
+      jb.img = const_cast<uint8_t *>(tc_wimg(ctx, kind, gph_tslot(c, j)));
+      jb.fexp = const_cast<int *>(tc_wfexp(ctx, kind, gph_tslot(c, j)));
+      jobs.push_back(jb);
     }
   }
   // job table: pointers are fixed for the ctx, re-uploaded only with the images
@@ -1786,6 +1791,8 @@ int tc_prepare_weights(occu_ctx *ctx, cudaStream_t st) {
   ctx->wimg_version = ctx->params_version;
   return 1;
 }
+
+int gph_tslot(const occu_config &c, int j) { return c.L + 1 + c.graphormer + j; }
 
 bool tc_supported(const occu_config &c) {
   return (c.d == 64 || c.d == 128) && c.F_n <= 128;
@@ -1970,6 +1977,24 @@ static int plain_impl(const occu_ctx *ctx, const float *A, int K, int R, int wki
   r.wimg = tc_wimg(ctx, wkind, layer); r.wfexp = tc_wfexp(ctx, wkind, layer);
   r.mask_h = mask_h; r.in_ptr = in_ptr; r.mean = ctx->cfg.aggr == OCCU_AGGR_MEAN;
   return launch_rowgemm<D, EPI_PLAIN>(ctx, r, name, st);
+}
+template <int D>
+static int plain_masked_impl(const occu_ctx *ctx, const float *A, int K, int R, int wkind, int layer,
+                             const float *add, float *out, const char *name, cudaStream_t st,
+                             const float *mask, float slope) {
+  RowGemmArgs r{};
+  r.slope = slope;
+  r.A = A; r.K = K; r.R = R; r.add = add; r.out = out;
+  r.wimg = tc_wimg(ctx, wkind, layer); r.wfexp = tc_wfexp(ctx, wkind, layer);
+  r.mask_h = mask; r.mean = 0;
+  return launch_rowgemm<D, EPI_PLAIN>(ctx, r, name, st);
+}
+int launch_plain_masked_tc(const occu_ctx *ctx, const float *A, int K, int R, int wkind, int layer,
+                           const float *add, float *out, const char *name, cudaStream_t st,
+                           const float *mask, float slope) {
+  if (R <= 0) return 0;
+  return ctx->cfg.d == 64 ? plain_masked_impl<64>(ctx, A, K, R, wkind, layer, add, out, name, st, mask, slope)
+                          : plain_masked_impl<128>(ctx, A, K, R, wkind, layer, add, out, name, st, mask, slope);
 }
 template <int D>
 static int bias_impl(const occu_ctx *ctx, const float *A, int K, int R, int wkind, int layer,

@@ -71,6 +71,9 @@ struct Workspace {
   DevBuf scsr, snf, sef, sdesc;   // occu_synthesize: batch CSR, node / edge rows, descriptors
   DevBuf hf;               // OCCU_BF16 with Graphormer / decoder: h_L widened to FP32 (R41)
   DevBuf gx, gqkv, go;     // Graphormer scratch: LN output [N][d], Q|K|V [3][N][d], attention [N][d]
+  std::vector<DevBuf> gsave;   // training: 8 saved [N][d] intermediates per Graphormer layer
+  DevBuf gscr;             // training: Graphormer backward scratch 5 x [N][d] + stats
+  DevBuf gdh[2];           // training: gradients w.r.t. the stack's node states (ping-pong)
   void release_all();
 };
 
@@ -246,8 +249,27 @@ int launch_bf16_to_f32(const occu_ctx *ctx, const void *src, size_t n, float *ds
 bool small_forward_ok(const occu_ctx *ctx, const DevCsr &csr);
 int launch_small_forward(const occu_ctx *ctx, const DevCsr &csr, const float *nf, const float *ef,
                          float *r, float *cvec, float *yhat, cudaStream_t st);
+// Graphormer layer intermediates kept for the backward (training): LN1 output, Q, K, V, the
+// attention output (before W_o), h̄, LN2 output, FFN hidden (post-ReLU), all [N][d].
+struct GphSave { float *X1, *Q, *K, *V, *O, *Hb, *X2, *T; };
 int launch_graphormer_layer(const occu_ctx *ctx, const DevCsr &csr, int j, const float *h_in,
-                            float *h_out, float *X, float *QKV, float *O, cudaStream_t st);
+                            float *h_out, float *X, float *QKV, float *O, cudaStream_t st,
+                            const GphSave *sv = nullptr);
+// Backward of Graphormer layer j (kernels_stack.cu): dout = ∂L/∂(layer output) -> dh_in
+// (∂L/∂h_in), parameter gradients into ctx->grads.  scratch: 5 x [N][d].
+int launch_graphormer_layer_bwd(occu_ctx *ctx, const DevCsr &csr, int j, const float *h_in,
+                                const GphSave &sv, const float *dout, float *dh_in, float *scratch,
+                                cudaStream_t st);
+// dA = dh ⊙ LReLU'(h) (÷ deg for MEAN), the last ANEE layer's aggregation gradient from the
+// gradient of its output h (kernels_stack.cu).
+int launch_mask_dA(const occu_ctx *ctx, const DevCsr &csr, const float *dh, const float *h, float *dA,
+                   cudaStream_t st);
+// Row-GEMM out = (A Wᵀ [+ add]) ⊙ (mask > 0 ? 1 : slope) with a prebuilt image (no ÷deg).
+int launch_plain_masked_tc(const occu_ctx *ctx, const float *A, int K, int R, int wkind, int layer,
+                           const float *add, float *out, const char *name, cudaStream_t st,
+                           const float *mask, float slope);
+// Image slot of Graphormer layer j's transposed matrices (kinds 0-5: W_qᵀ W_kᵀ W_vᵀ W_oᵀ W1ᵀ W2ᵀ).
+int gph_tslot(const occu_config &c, int j);
 int launch_bias_add_tc(const occu_ctx *ctx, const float *A, int K, int R, int wkind, int layer,
                        const float *bias, const float *add, float *out, const char *name,
                        cudaStream_t st);

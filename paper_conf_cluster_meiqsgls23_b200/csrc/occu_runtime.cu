@@ -50,10 +50,10 @@ void Workspace::release_all() {
   DevBuf *bufs[] = {&node_feat, &edge_feat, &targets, &out_occ, &csr, &e0, &g, &r, &c, &yhat,
                     &dy, &dc, &dr, &dh, &dhprev, &dP, &MG, &DV, &DZ, &deA, &deB, &dalpha,
                     &dpq, &partial, &loss, &tcpart, &dpart, &rpart, &anf[0], &anf[1],
-                    &aef[0], &aef[1], &acsr[0], &acsr[1], &dT, &dZ, &dprep, &dpool, &gx, &gqkv, &go,
+                    &aef[0], &aef[1], &acsr[0], &acsr[1], &dT, &dZ, &dprep, &dpool, &gx, &gqkv, &go, &gscr, &gdh[0], &gdh[1],
                     &scsr, &snf, &sef, &sdesc, &hf};
   for (DevBuf *b : bufs) b->release();
-  for (auto *v : {&hbar, &p, &q, &e, &h, &gs, &gh})
+  for (auto *v : {&hbar, &p, &q, &e, &h, &gs, &gh, &gsave})
     for (DevBuf &b : *v) b.release();
 }
 
@@ -339,10 +339,19 @@ occu_status forward(occu_ctx *ctx, const DevCsr &csr, const float *nf, const flo
     CK(w.gx.ensure(size_t(csr.N) * c.d * 4), "alloc graphormer scratch");
     CK(w.gqkv.ensure(size_t(csr.N) * 3 * c.d * 4), "alloc graphormer scratch");
     CK(w.go.ensure(size_t(csr.N) * c.d * 4), "alloc graphormer scratch");
+    if (save_all) {                     // training: every intermediate kept for the backward
+      if (w.gsave.size() < size_t(8 * c.graphormer)) w.gsave.resize(8 * c.graphormer);
+      for (auto &b : w.gsave) CK(b.ensure(size_t(csr.N) * c.d * 4), "alloc graphormer saves");
+    }
     for (int j = 0; j < c.graphormer; ++j) {
       float *out = w.gh[j].as<float>();
+      GphSave sv;
+      if (save_all) {
+        float **f[8] = {&sv.X1, &sv.Q, &sv.K, &sv.V, &sv.O, &sv.Hb, &sv.X2, &sv.T};
+        for (int t = 0; t < 8; ++t) *f[t] = w.gsave[8 * j + t].as<float>();
+      }
       LK(launch_graphormer_layer(ctx, csr, j, h_top, out, w.gx.as<float>(), w.gqkv.as<float>(),
-                                 w.go.as<float>(), s),
+                                 w.go.as<float>(), s, save_all ? &sv : nullptr),
          "graphormer layer");
       h_top = out;
     }
@@ -413,10 +422,11 @@ occu_status grads_impl(occu_ctx *ctx, const occu_batch *batch, const float *targ
   if (!batch || !batch->csr || !targets) return fail(ctx, OCCU_EINVAL, "batch/targets NULL");
   if (batch->global_num_graphs < batch->csr->num_graphs)
     return fail(ctx, OCCU_EINVAL, "global_num_graphs < local num_graphs");
+  const bool stack = ctx->cfg.readout == OCCU_READOUT_SET_DECODER || ctx->cfg.graphormer > 0;
+  if (stack && (ctx->cfg.prec != OCCU_FP32 || ctx->path != 0))
+    return fail(ctx, OCCU_EINVAL, "training through the Graphormer layers / decoder readout runs in OCCU_FP32 on kernel path 0");
   if (ctx->cfg.readout == OCCU_READOUT_SET_DECODER)
     return fail(ctx, OCCU_EINVAL, "the Set-Transformer decoder readout is inference-only in this build");
-  if (ctx->cfg.graphormer > 0)
-    return fail(ctx, OCCU_EINVAL, "Graphormer layers are inference-only in this build");
   if (ctx->cfg.msg == OCCU_MSG_NEIGHBOR_SOFTMAX && ctx->cfg.prec == OCCU_BF16)
     return fail(ctx, OCCU_EINVAL, "reading B in OCCU_BF16 is inference-only in this build");
   ctx->launches = 0;
@@ -443,6 +453,27 @@ occu_status grads_impl(occu_ctx *ctx, const occu_batch *batch, const float *targ
   CK(w.loss.ensure(4), "alloc");
   cudaStream_t s = ctx->stream;
   LK(launch_head_backward(ctx, csr, stg.y, batch->global_num_graphs, s), "head backward");
+  if (stack) {
+    // NEXT-2 / NEXT-3 training: ∂L/∂(stack top) from the readout, then the Graphormer layers in
+    // reverse, then dA of the last ANEE layer (what the ANEE backward consumes in w.dh)
+    for (auto &b : w.gdh) CK(b.ensure(Nd), "alloc stack gradients");
+    const size_t scr = 5 * Nd + size_t(csr.N) * std::max(c.heads, 1) * 12;
+    CK(w.gscr.ensure(scr), "alloc stack scratch");
+    float *g = w.gdh[0].as<float>();
+    // mean readout: broadcast_dh (launched by the head backward without a mask) left dr/n_b
+    CK(cudaMemcpyAsync(g, w.dh.ptr, Nd, cudaMemcpyDeviceToDevice, s), "copy dh");
+    for (int j = c.graphormer - 1; j >= 0; --j) {
+      const float *hin = j == 0 ? w.h[c.L - 1].as<float>() : w.gh[j - 1].as<float>();
+      GphSave sv;
+      float **f[8] = {&sv.X1, &sv.Q, &sv.K, &sv.V, &sv.O, &sv.Hb, &sv.X2, &sv.T};
+      for (int t = 0; t < 8; ++t) *f[t] = w.gsave[8 * j + t].as<float>();
+      float *gout = w.gdh[(c.graphormer - j) & 1].as<float>();
+      LK(launch_graphormer_layer_bwd(ctx, csr, j, hin, sv, g, gout, w.gscr.as<float>(), s),
+         "graphormer backward");
+      g = gout;
+    }
+    LK(launch_mask_dA(ctx, csr, g, w.h[c.L - 1].as<float>(), w.dh.as<float>(), s), "mask dA");
+  }
   for (int i = c.L - 1; i >= 0; --i) {
     BwdLayerArgs a{};
     a.layer = i;

@@ -160,8 +160,10 @@ def test_graphormer_errors():
     with pytest.raises(occu.OccuError):
         m.set_kernel_path(1)
     b = configs.random_dag_batch(3, 5, max_nodes=10)
-    with pytest.raises(occu.OccuError):
-        m.train_step(occu.pack(b.graphs), b.node_feat, b.edge_feat, b.targets, 1e-4)
+    mb = occu.Model(occu.config(L=2, d=64, prec=occu.BF16, graphormer=1, heads=2))
+    mb.init_weights(1)
+    with pytest.raises(occu.OccuError):          # training through the stack: OCCU_FP32 only
+        mb.train_step(occu.pack(b.graphs), b.node_feat, b.edge_feat, b.targets, 1e-4)
 
 
 def test_graphormer_parity_is_sensitive_to_the_attention():
@@ -210,3 +212,44 @@ def test_bf16_anee_with_fp32_graphormer_and_decoder(G, readout, msg):
     yr = oracle.forward(params, ocfg(c), pk, b.node_feat, b.edge_feat)["yhat"]
     assert rel(y, yr) <= 1e-2
     assert np.all(np.abs(y - yr) <= 1e-2 * np.maximum(np.abs(yr), 0.1)), np.abs(y - yr).max()
+
+
+# ---------------------------------------------------------------- training (NEXT-3)
+@pytest.mark.parametrize("L,d,G,heads,aggr", [(2, 64, 1, 2, 0), (3, 128, 2, 4, 0), (2, 128, 2, 8, 1),
+                                              (2, 64, 2, 4, 0)])
+def test_graphormer_training_gradients_match_oracle(L, d, G, heads, aggr):
+    """Training through the Graphormer layers (the paper's encoder, P153-P157 + P273's Adam):
+    the loss and every per-tensor gradient — ANEE, Graphormer (LN, Q/K/V/O, FFN), head —
+    against the float64 oracle's hand-derived backward (itself pinned by torch autograd and
+    finite differences), rel-L2 <= 1e-4."""
+    c = mk(L, d, G, heads, aggr=aggr)
+    b = with_single(configs.random_dag_batch(20, 7100 + L + G + heads, max_nodes=90, hub=True))
+    flat = params_for(c, 40 + G)
+    m = occu.Model(c)
+    m.set_params(flat)
+    loss = m.compute_grads(occu.pack(b.graphs), b.node_feat, b.edge_feat, b.targets,
+                           global_num_graphs=32)
+    g = weights.unflatten(wcfg(c), m.get_grads())
+    params = oracle.unflatten(ocfg(c), flat.astype(np.float64))
+    lref, gref = oracle.loss_and_grads(params, ocfg(c), b.graphs, b.node_feat, b.edge_feat,
+                                       b.targets, global_batch=32)
+    assert abs(loss - lref) <= TOL * abs(lref)
+    bad = {k: rel(g[k], gref[k]) for k in gref if rel(g[k], gref[k]) > TOL}
+    assert not bad, bad
+
+
+def test_graphormer_training_trajectory():
+    """Ten Adam steps through the stack track the oracle's loss trajectory."""
+    c = mk(2, 64, 1, 2)
+    b = configs.random_dag_batch(12, 7200, max_nodes=40, hub=True)
+    flat = params_for(c, 44)
+    m = occu.Model(c)
+    m.set_params(flat)
+    csr = occu.pack(b.graphs)
+    params = oracle.unflatten(ocfg(c), flat.astype(np.float64))
+    st = {}
+    for step in range(10):
+        loss = m.train_step(csr, b.node_feat, b.edge_feat, b.targets, 1e-3)
+        lref, gref = oracle.loss_and_grads(params, ocfg(c), b.graphs, b.node_feat, b.edge_feat, b.targets)
+        params, st = oracle.adam_step(params, gref, st, 1e-3)
+        assert abs(loss - lref) <= TOL * abs(lref) + 1e-7, (step, loss, lref)
