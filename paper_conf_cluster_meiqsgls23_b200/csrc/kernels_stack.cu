@@ -11,8 +11,9 @@
 //     dT = (dout W2) ⊙ [T > 0]; dX2 = dT W1; dh̄ = dout + LN2ᵀ(dX2); dO = dh̄ W_o;
 //     attention backward per graph and head (below); dX1 = dQ W_q + dK W_k + dV W_v;
 //     dH = dh̄ + LN1ᵀ(dX1).
-//   Attention backward (FP32 CUDA cores, two passes, no atomics): stats m_i, l_i of every
-//   query row over its own graph's keys and D_i = <dO_i, O_i>; then
+//   Attention backward (FP32 CUDA cores, no atomics): stats m_i, l_i of every query row over
+//   its own graph's keys and D_i = Σ_j P_ij (dO_i·V_j) (= <dO_i, O_i>, from the recomputed P,
+//   taken relative to the dominant key so that saturated softmax rows do not cancel);
 //     dQ_i = Σ_j P_ij (dO_i·V_j − D_i) K_j / √d_h        (thread = query row)
 //     dV_j = Σ_i P_ij dO_i,  dK_j = Σ_i P_ij (dO_i·V_j − D_i) Q_i / √d_h   (thread = key row)
 //   with P_ij = exp(s_ij − m_i)/l_i recomputed, keys / queries of the block's graphs staged
@@ -20,6 +21,8 @@
 #include <cuda_runtime.h>
 #include <math.h>
 #include <stdint.h>
+#include <stdio.h>
+#include <stdlib.h>
 
 #include <algorithm>
 
@@ -184,7 +187,7 @@ struct AttnBwdArgs {
   const float *Q, *K, *V, *O, *dO;   // [N][D]
   const int32_t *node_off, *node_graph;
   float *dQ, *dK, *dV;               // [N][D]
-  float *stats;                      // [N][heads][3]: m, l, D
+  float *stats;                      // [N][heads][4]: m, l, D', dP_ir (see pass 2)
   int N, D, heads;
   float scale;                       // 1 / sqrt(d_h)
 };
@@ -205,7 +208,6 @@ __global__ void __launch_bounds__(ABT) attn_bwd_q_kernel(const AttnBwdArgs a) {
   const int ub = __ldg(a.node_off + b0), ue = __ldg(a.node_off + b1 + 1);   // union key range
   int kb = 0, ke = 0;
   float q[DH], go[DH], acc[DH];
-  float Di = 0.f;
   if (live) {
     const int b = __ldg(a.node_graph + i);
     kb = __ldg(a.node_off + b);
@@ -214,12 +216,12 @@ __global__ void __launch_bounds__(ABT) attn_bwd_q_kernel(const AttnBwdArgs a) {
     for (int c = 0; c < DH; ++c) {
       q[c] = __ldg(a.Q + i * a.D + h * DH + c) * a.scale;
       go[c] = __ldg(a.dO + i * a.D + h * DH + c);
-      Di = fmaf(go[c], __ldg(a.O + i * a.D + h * DH + c), Di);
       acc[c] = 0.f;
     }
   }
   // pass 1: row maximum and normaliser over the own graph's keys
   float m = -INFINITY, l = 0.f;
+  int ref = kb;                                  // first key attaining the row maximum
   for (int t0 = ub; t0 < ue; t0 += TK) {
     __syncthreads();
     for (int e = threadIdx.x; e < TK * DH; e += ABT) {
@@ -236,6 +238,7 @@ __global__ void __launch_bounds__(ABT) attn_bwd_q_kernel(const AttnBwdArgs a) {
         if (s > m) {
           l = l * expf(m - s) + 1.f;
           m = s;
+          ref = j;
         } else {
           l += expf(s - m);
         }
@@ -243,7 +246,43 @@ __global__ void __launch_bounds__(ABT) attn_bwd_q_kernel(const AttnBwdArgs a) {
     }
   }
   const float inv_l = 1.f / l;
-  // pass 2: dQ
+  // pass 2: D_i = Σ_j P_ij dP_ij taken relative to the dominant key r (the first one at the
+  // row maximum): D'_i = Σ_j P_ij (dP_ij − dP_ir) and dS_ij = P_ij ((dP_ij − dP_ir) − D'_i).
+  // Same value as P ⊙ (dP − D), but when the softmax saturates (P_ir -> 1) the plain form
+  // cancels dP_ir − D ≈ (1 − P_ir)·Δ at a rounding error ~ε|dP_ir| while this form keeps
+  // ~ε|Δ| (float64 accumulation, the recomputed P).
+  float dpr = 0.f, Dp = 0.f;
+  if (live) {
+#pragma unroll
+    for (int c = 0; c < DH; ++c) dpr = fmaf(go[c], __ldg(a.V + long(ref) * a.D + h * DH + c), dpr);
+  }
+  {
+    double dacc = 0.0;
+    for (int t0 = ub; t0 < ue; t0 += TK) {
+      __syncthreads();
+      for (int e = threadIdx.x; e < TK * DH; e += ABT) {
+        const int rr = e / DH, cc = e % DH;
+        const bool in = t0 + rr < ue;
+        sk[rr][cc] = in ? __ldg(a.K + long(t0 + rr) * a.D + h * DH + cc) : 0.f;
+        sv[rr][cc] = in ? __ldg(a.V + long(t0 + rr) * a.D + h * DH + cc) : 0.f;
+      }
+      __syncthreads();
+      if (live) {
+        const int jb = max(kb, t0), je = min(ke, t0 + TK);
+        for (int j = jb; j < je; ++j) {
+          float s = 0.f, dp = 0.f;
+#pragma unroll
+          for (int c = 0; c < DH; ++c) {
+            s = fmaf(q[c], sk[j - t0][c], s);
+            dp = fmaf(go[c], sv[j - t0][c], dp);
+          }
+          dacc = fma(double(expf(s - m) * inv_l), double(dp - dpr), dacc);
+        }
+      }
+    }
+    Dp = float(dacc);
+  }
+  // pass 3: dQ
   for (int t0 = ub; t0 < ue; t0 += TK) {
     __syncthreads();
     for (int e = threadIdx.x; e < TK * DH; e += ABT) {
@@ -263,7 +302,7 @@ __global__ void __launch_bounds__(ABT) attn_bwd_q_kernel(const AttnBwdArgs a) {
           dp = fmaf(go[c], sv[j - t0][c], dp);
         }
         const float p = expf(s - m) * inv_l;
-        const float ds = p * (dp - Di);
+        const float ds = p * ((dp - dpr) - Dp);
 #pragma unroll
         for (int c = 0; c < DH; ++c) acc[c] = fmaf(ds, sk[j - t0][c], acc[c]);
       }
@@ -272,17 +311,18 @@ __global__ void __launch_bounds__(ABT) attn_bwd_q_kernel(const AttnBwdArgs a) {
   if (live) {
 #pragma unroll
     for (int c = 0; c < DH; ++c) a.dQ[i * a.D + h * DH + c] = acc[c] * a.scale;
-    float *stt = a.stats + (i * a.heads + h) * 3;
+    float *stt = a.stats + (i * a.heads + h) * 4;
     stt[0] = m;
     stt[1] = l;
-    stt[2] = Di;
+    stt[2] = Dp;
+    stt[3] = dpr;
   }
 }
 
 // dK, dV: thread = key row j of head blockIdx.y; queries of the block's graphs staged.
 template <int DH>
 __global__ void __launch_bounds__(ABT) attn_bwd_kv_kernel(const AttnBwdArgs a) {
-  __shared__ float sq[TK][DH], sg[TK][DH], ss[TK][3];
+  __shared__ float sq[TK][DH], sg[TK][DH], ss[TK][4];
   const int h = blockIdx.y;
   const long j0 = long(blockIdx.x) * ABT;
   const long j = j0 + threadIdx.x;
@@ -311,9 +351,9 @@ __global__ void __launch_bounds__(ABT) attn_bwd_kv_kernel(const AttnBwdArgs a) {
       sq[rr][cc] = in ? __ldg(a.Q + long(t0 + rr) * a.D + h * DH + cc) * a.scale : 0.f;
       sg[rr][cc] = in ? __ldg(a.dO + long(t0 + rr) * a.D + h * DH + cc) : 0.f;
     }
-    for (int e = threadIdx.x; e < TK * 3; e += ABT) {
-      const int rr = e / 3, cc = e % 3;
-      ss[rr][cc] = t0 + rr < ue ? a.stats[(long(t0 + rr) * a.heads + h) * 3 + cc] : 1.f;
+    for (int e = threadIdx.x; e < TK * 4; e += ABT) {
+      const int rr = e / 4, cc = e % 4;
+      ss[rr][cc] = t0 + rr < ue ? a.stats[(long(t0 + rr) * a.heads + h) * 4 + cc] : 1.f;
     }
     __syncthreads();
     if (live) {
@@ -327,7 +367,7 @@ __global__ void __launch_bounds__(ABT) attn_bwd_kv_kernel(const AttnBwdArgs a) {
           dp = fmaf(sg[r][c], v[c], dp);
         }
         const float p = expf(s - ss[r][0]) / ss[r][1];
-        const float ds = p * (dp - ss[r][2]);
+        const float ds = p * ((dp - ss[r][3]) - ss[r][2]);
 #pragma unroll
         for (int c = 0; c < DH; ++c) {
           dv[c] = fmaf(p, sg[r][c], dv[c]);
@@ -403,7 +443,7 @@ int launch_graphormer_layer_bwd(occu_ctx *ctx, const DevCsr &csr, int j, const f
   const size_t ND = size_t(N) * D;
   float *s1 = scratch, *s2 = scratch + ND, *s3 = scratch + 2 * ND, *s4 = scratch + 3 * ND,
         *s5 = scratch + 4 * ND;
-  float *stats = scratch + 5 * ND;                        // [N][heads][3]
+  float *stats = scratch + 5 * ND;                        // [N][heads][4]
   int n = 0, r;
 #define SKR(call)                  \
   do {                             \

@@ -457,7 +457,7 @@ occu_status grads_impl(occu_ctx *ctx, const occu_batch *batch, const float *targ
     // NEXT-2 / NEXT-3 training: ∂L/∂(stack top) from the readout, then the Graphormer layers in
     // reverse, then dA of the last ANEE layer (what the ANEE backward consumes in w.dh)
     for (auto &b : w.gdh) CK(b.ensure(Nd), "alloc stack gradients");
-    const size_t scr = 5 * Nd + size_t(csr.N) * std::max(c.heads, 1) * 12;
+    const size_t scr = 5 * Nd + size_t(csr.N) * std::max(c.heads, 1) * 16;
     CK(w.gscr.ensure(scr), "alloc stack scratch");
     float *g = w.gdh[0].as<float>();
     // mean readout: broadcast_dh (launched by the head backward without a mask) left dr/n_b
