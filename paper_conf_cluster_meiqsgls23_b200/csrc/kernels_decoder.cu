@@ -675,6 +675,555 @@ __global__ void __launch_bounds__(DT_TAIL) set_decoder_kernel(const DecArgs a, c
   }
 }
 
+// =========================================================================================
+// Training through the decoder readout (NEXT-2; oracle.set_decoder_bwd, R46).
+//
+// Per graph g (CTA per graph, dec_tail_bwd_kernel): the tail is recomputed from the pool
+// partials exactly as set_decoder_kernel forms it, every k-row intermediate kept in shared
+// memory, then the chain is differentiated backwards from dr = ∂L/∂(decoder output):
+//   FFN_D, SAB (= MAB2: LN2, FFN, LN1, W_o, the k x k attention per head, W_q/W_k/W_v),
+//   PMA's tail (MAB1: LN2, FFN, LN1, W_o)  ->  dO1 = ∂L/∂(W_v P̄ + b_v) per (seed, head).
+// Weight gradients need sums over graphs: each graph writes its (input, output-gradient) rows
+// to row arrays [B·k][d] and fixed-order row reductions (dec_rows_wgrad_kernel, column sums,
+// LayerNorm parameter sums) form them afterwards.  The node side (dec_pool_bwd_kernel) uses
+// the folded key map of the forward: score s_n = Z_n·M_kh + c_kh, α = softmax_n(s), so with
+// u_kh = W_v,hᵀ dO1_kh:  ∂α_n = Z_n·u_kh,  ds_n = α_n (∂α_n − Σ_m α_m ∂α_m),
+//   ∂Z_n = Σ_kh (α_n,kh u_kh + ds_n,kh M_kh),   G_kh = Σ_n ds_n,kh Z_n,  σ_kh = Σ_n ds_n,kh,
+// and the seeds' query gradient ∂q_kh = (W_k,h G_kh + b_k,h σ_kh)/√d_h, where σ_kh = 0 exactly
+// (so ∂b_k = 0); ∂α and G are formed relative to the graph's first node (dec_pool_bwd_kernel),
+// ∂W_k,h = Σ_j (q_jh/√d_h) ⊗ G_jh summed over graphs (dec_seed_grads_kernel).
+// =========================================================================================
+
+// Row-array slots written by dec_tail_bwd_kernel ([B·k][D] each).
+enum DecRow {
+  R_UD, R_dUD, R_sab, R_dsab, R_T4, R_U2, R_dU2, R_Hb2, R_dT4, R_dHb2, R_T3, R_O2, R_dT3,
+  R_dQ2, R_dK2, R_dV2, R_pma, R_dpma, R_T2, R_U1, R_dU1, R_Hb1, R_dT2, R_dHb1, R_T1, R_O1,
+  R_dT1, R_dO1, R_COUNT
+};
+
+// Y[v][c] (+)= Σ_n X[v][n] W[n·ldw + c] for c < ncols, n < nrows, v < nvec (transposed GEMV):
+// warps split the rows n, lane = 4 columns (coalesced W rows), warp partials summed in warp
+// order through shared memory (scratch [NW][nvec][ncols]).  Fixed order.
+__device__ void gemv_t(const float *__restrict__ W, int ldw, int nrows, int ncols, const float *X, int ldx,
+                       int nvec, float *Y, int ldy, float *scratch, bool acc) {
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, nw = blockDim.x >> 5;
+  const int per = (nrows + nw - 1) / nw, nb = warp * per, ne = min(nrows, nb + per);
+  for (int c0 = 0; c0 < ncols; c0 += 128) {
+    const int c = c0 + lane * 4;
+    float4 a[KMAX];
+#pragma unroll
+    for (int v = 0; v < KMAX; ++v) a[v] = make_float4(0.f, 0.f, 0.f, 0.f);
+    if (c < ncols)
+      for (int n = nb; n < ne; ++n) {
+        const float4 w = __ldg(reinterpret_cast<const float4 *>(W + long(n) * ldw + c));
+#pragma unroll
+        for (int v = 0; v < KMAX; ++v)
+          if (v < nvec) {
+            const float x = X[v * ldx + n];
+            a[v].x = fmaf(x, w.x, a[v].x); a[v].y = fmaf(x, w.y, a[v].y);
+            a[v].z = fmaf(x, w.z, a[v].z); a[v].w = fmaf(x, w.w, a[v].w);
+          }
+      }
+    if (c < ncols)
+#pragma unroll
+      for (int v = 0; v < KMAX; ++v)
+        if (v < nvec) *reinterpret_cast<float4 *>(scratch + (warp * KMAX + v) * 128 + lane * 4) = a[v];
+    __syncthreads();
+    for (int o = threadIdx.x; o < nvec * 128; o += blockDim.x) {
+      const int v = o / 128, cc = o % 128;
+      if (c0 + cc < ncols) {
+        float t = 0.f;
+        for (int w2 = 0; w2 < nw; ++w2) t += scratch[(w2 * KMAX + v) * 128 + cc];
+        float *y = Y + v * ldy + c0 + cc;
+        *y = acc ? *y + t : t;
+      }
+    }
+    __syncthreads();
+  }
+}
+
+// LayerNorm backward per vector (warp per vector): x = the LN input rows, dy = ∂L/∂y;
+// dx (=, or += with acc) rstd·(g⊙dy − mean(g⊙dy) − x̂·mean(g⊙dy⊙x̂)).
+template <int D>
+__device__ void warp_ln_bwd(const float *x, const float *dy, float *dx, int nvec,
+                            const float *__restrict__ g, bool acc) {
+  constexpr int V = D / 32;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, nw = blockDim.x >> 5;
+  for (int v = warp; v < nvec; v += nw) {
+    float xv[V], s = 0.f;
+#pragma unroll
+    for (int i = 0; i < V; ++i) {
+      xv[i] = x[v * D + lane + 32 * i];
+      s += xv[i];
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+    const float mu = s / float(D);
+    float q = 0.f;
+#pragma unroll
+    for (int i = 0; i < V; ++i) q = fmaf(xv[i] - mu, xv[i] - mu, q);
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) q += __shfl_xor_sync(0xffffffffu, q, o);
+    const float rstd = rsqrtf(q / float(D) + 1e-5f);
+    float a1 = 0.f, a2 = 0.f, xh[V], gd[V];
+#pragma unroll
+    for (int i = 0; i < V; ++i) {
+      const int ch = lane + 32 * i;
+      xh[i] = (xv[i] - mu) * rstd;
+      gd[i] = g[ch] * dy[v * D + ch];
+      a1 += gd[i];
+      a2 = fmaf(gd[i], xh[i], a2);
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+      a1 += __shfl_xor_sync(0xffffffffu, a1, o);
+      a2 += __shfl_xor_sync(0xffffffffu, a2, o);
+    }
+    a1 /= float(D);
+    a2 /= float(D);
+#pragma unroll
+    for (int i = 0; i < V; ++i) {
+      const int ch = lane + 32 * i;
+      const float o = rstd * (gd[i] - a1 - xh[i] * a2);
+      dx[v * D + ch] = acc ? dx[v * D + ch] + o : o;
+    }
+  }
+}
+
+struct DecBwdArgs {
+  DecArgs f;                     // forward arguments (weights, layout, sizes)
+  const float *part;             // pool partials of the forward
+  const float *dr;               // [B][k·D] ∂L/∂(decoder output)
+  float *rows;                   // [R_COUNT][B·k][D]
+  float *pstat;                  // [B][KHMAX][2]: merged pool max, sum
+  float *pbar;                   // [B·k·heads][D] merged pooled Z (P̄)
+  float *u;                      // [B][KHMAX][D]: W_v,hᵀ dO1_kh
+};
+
+template <int D>
+constexpr size_t tail_bwd_smem_floats() {
+  return size_t(NPV) * D + size_t(KMAX) * D + size_t(KHMAX) * D + 2 * KHMAX + SPLIT * KHMAX +
+         size_t(KMAX) * KMAX * 8 * 2 + size_t(30) * KMAX * D + size_t(NW) * KMAX * 128;
+}
+
+template <int D>
+__global__ void __launch_bounds__(DT_TAIL) dec_tail_bwd_kernel(const DecBwdArgs b) {
+  extern __shared__ __align__(16) float sm[];
+  const DecArgs &a = b.f;
+  const int k = a.k, heads = a.heads, KH = k * heads, dh = D / heads;
+  const int g = blockIdx.x, t = threadIdx.x;
+  const DecLayout &L = a.L;
+  const float *P = a.P;
+  const float isq = rsqrtf(float(dh));
+  float *pv = sm;                                  // [NPV][D]
+  float *Ssm = pv + NPV * D;                       // [KMAX][D] seeds
+  float *Pacc = Ssm + KMAX * D;                    // [KHMAX][D]
+  float *mstat = Pacc + KHMAX * D, *lsum = mstat + KHMAX;
+  float *fs = lsum + KHMAX;                        // [SPLIT][KHMAX]
+  float *Watt = fs + SPLIT * KHMAX;                // [heads][k][k] (max 8 x 8 x 8)
+  float *dWatt = Watt + KMAX * KMAX * 8;
+  float *buf = dWatt + KMAX * KMAX * 8;            // 30 x [KMAX][D]
+  float *scr = buf + 30 * KMAX * D;                // gemv_t scratch [NW][KMAX][128]
+  auto B = [&](int i) { return buf + i * KMAX * D; };
+  const size_t vo[NPV] = {L.M1.bv, L.M1.bo, L.M1.ln1_g, L.M1.ln1_b, L.M1.F.b1, L.M1.F.b2,
+                          L.M1.ln2_g, L.M1.ln2_b, L.M2.bq, L.M2.bk, L.M2.bv, L.M2.bo,
+                          L.M2.ln1_g, L.M2.ln1_b, L.M2.F.b1, L.M2.F.b2, L.M2.ln2_g, L.M2.ln2_b,
+                          L.D.b1, L.D.b2};
+  for (int i = t; i < NPV * D; i += DT_TAIL) pv[i] = __ldg(P + vo[i / D] + i % D);
+  for (int i = t; i < k * D; i += DT_TAIL) Ssm[i] = __ldg(P + L.S + i);
+  auto PV = [&](int i) -> const float * { return pv + i * D; };
+  constexpr int PS = part_stride<D>();
+  const float *pg = b.part + long(g) * SPLIT * PS;
+  for (int kh = t; kh < KH; kh += DT_TAIL) {       // merge exactly as set_decoder_kernel
+    float M = -INFINITY;
+    for (int q = 0; q < SPLIT; ++q) M = fmaxf(M, pg[q * PS + KHMAX * D + kh]);
+    float l = 0.f;
+    for (int q = 0; q < SPLIT; ++q) {
+      const float mq = pg[q * PS + KHMAX * D + kh];
+      const float f = mq == -INFINITY ? 0.f : ex2((mq - M) * L2E);
+      fs[q * KHMAX + kh] = f;
+      l = fmaf(pg[q * PS + KHMAX * D + KHMAX + kh], f, l);
+    }
+    mstat[kh] = M;
+    lsum[kh] = l;
+    b.pstat[(long(g) * KHMAX + kh) * 2] = M;
+    b.pstat[(long(g) * KHMAX + kh) * 2 + 1] = l;
+  }
+  __syncthreads();
+  for (int o = t; o < KH * D; o += DT_TAIL) {
+    const int kh = o / D;
+    float acc = 0.f;
+    for (int q = 0; q < SPLIT; ++q) acc = fmaf(pg[q * PS + o], fs[q * KHMAX + kh], acc);
+    Pacc[o] = acc / lsum[kh];
+    b.pbar[long(g) * KH * D + o] = Pacc[o];
+  }
+  __syncthreads();
+  // ---- forward recompute (set_decoder_kernel's chain), every intermediate kept
+  float *O1 = B(0), *A1 = B(1), *T1 = B(2), *Hb1 = B(3), *U1 = B(4), *F1 = B(5), *T2 = B(6),
+        *pma = B(7), *Q2 = B(8), *K2 = B(9), *V2 = B(10), *O2 = B(11), *A2 = B(12), *T3 = B(13),
+        *Hb2 = B(14), *U2 = B(15), *F2 = B(16), *T4 = B(17), *sab = B(18), *UD = B(19);
+  float *g0 = B(20), *g1 = B(21), *g2 = B(22), *g3 = B(23), *g4 = B(24), *g5 = B(25), *g6 = B(26),
+        *g7 = B(27), *g8 = B(28), *g9 = B(29);
+  const int V = k;
+  for (int h = 0; h < heads; ++h)
+    gemv_k(P + L.M1.Wv + long(h) * dh * D, D, D, dh, Pacc + h * D, heads * D, V, O1 + h * dh, D,
+           PV(0) + h * dh, false);
+  __syncthreads();
+  gemv_k(P + L.M1.Wo, D, D, D, O1, D, V, A1, D, PV(1), false);
+  __syncthreads();
+  for (int i = t; i < V * D; i += DT_TAIL) T1[i] = Ssm[i] + A1[i];
+  __syncthreads();
+  warp_add_ln<D>(Ssm, A1, Hb1, V, PV(2), PV(3));
+  __syncthreads();
+  gemv_k(P + L.M1.F.W1, D, D, D, Hb1, D, V, U1, D, PV(4), true);
+  __syncthreads();
+  gemv_k(P + L.M1.F.W2, D, D, D, U1, D, V, F1, D, PV(5), false);
+  __syncthreads();
+  for (int i = t; i < V * D; i += DT_TAIL) T2[i] = Hb1[i] + F1[i];
+  warp_add_ln<D>(Hb1, F1, pma, V, PV(6), PV(7));
+  __syncthreads();
+  gemv_k(P + L.M2.Wq, D, D, D, pma, D, V, Q2, D, PV(8), false);
+  gemv_k(P + L.M2.Wk, D, D, D, pma, D, V, K2, D, PV(9), false);
+  gemv_k(P + L.M2.Wv, D, D, D, pma, D, V, V2, D, PV(10), false);
+  __syncthreads();
+  const int KK = k * k;
+  for (int o = t; o < heads * KK; o += DT_TAIL) {
+    const int h = o / KK, j = (o / k) % k, jj = o % k;
+    float sdot = 0.f;
+    for (int i = 0; i < dh; ++i) sdot = fmaf(Q2[j * D + h * dh + i], K2[jj * D + h * dh + i], sdot);
+    Watt[o] = sdot * isq;
+  }
+  __syncthreads();
+  for (int o = t; o < heads * k; o += DT_TAIL) {
+    float m = -INFINITY, l = 0.f;
+    for (int jj = 0; jj < k; ++jj) m = fmaxf(m, Watt[o * k + jj]);
+    for (int jj = 0; jj < k; ++jj) {
+      const float w = ex2((Watt[o * k + jj] - m) * L2E);
+      Watt[o * k + jj] = w;
+      l += w;
+    }
+    for (int jj = 0; jj < k; ++jj) Watt[o * k + jj] /= l;
+  }
+  __syncthreads();
+  for (int o = t; o < V * D; o += DT_TAIL) {
+    const int j = o / D, ch = o % D, h = ch / dh;
+    const float *w = Watt + (h * k + j) * k;
+    float acc = 0.f;
+    for (int jj = 0; jj < k; ++jj) acc = fmaf(w[jj], V2[jj * D + ch], acc);
+    O2[o] = acc;
+  }
+  __syncthreads();
+  gemv_k(P + L.M2.Wo, D, D, D, O2, D, V, A2, D, PV(11), false);
+  __syncthreads();
+  for (int i = t; i < V * D; i += DT_TAIL) T3[i] = pma[i] + A2[i];
+  warp_add_ln<D>(pma, A2, Hb2, V, PV(12), PV(13));
+  __syncthreads();
+  gemv_k(P + L.M2.F.W1, D, D, D, Hb2, D, V, U2, D, PV(14), true);
+  __syncthreads();
+  gemv_k(P + L.M2.F.W2, D, D, D, U2, D, V, F2, D, PV(15), false);
+  __syncthreads();
+  for (int i = t; i < V * D; i += DT_TAIL) T4[i] = Hb2[i] + F2[i];
+  warp_add_ln<D>(Hb2, F2, sab, V, PV(16), PV(17));
+  __syncthreads();
+  gemv_k(P + L.D.W1, D, D, D, sab, D, V, UD, D, PV(18), true);
+  __syncthreads();
+  // ---- backward
+  const float *dD = b.dr + long(g) * k * D;
+  for (int i = t; i < V * D; i += DT_TAIL) g9[i] = dD[i];
+  __syncthreads();
+  gemv_t(P + L.D.W2, D, D, D, g9, D, V, g0, D, scr, false);        // ∂UD
+  __syncthreads();
+  for (int i = t; i < V * D; i += DT_TAIL) g0[i] = UD[i] > 0.f ? g0[i] : 0.f;
+  __syncthreads();
+  gemv_t(P + L.D.W1, D, D, D, g0, D, V, g1, D, scr, false);        // ∂sab
+  __syncthreads();
+  warp_ln_bwd<D>(T4, g1, g2, V, PV(16), false);                    // ∂T4 (= ∂F2)
+  __syncthreads();
+  gemv_t(P + L.M2.F.W2, D, D, D, g2, D, V, g3, D, scr, false);     // ∂U2
+  __syncthreads();
+  for (int i = t; i < V * D; i += DT_TAIL) g3[i] = U2[i] > 0.f ? g3[i] : 0.f;
+  for (int i = t; i < V * D; i += DT_TAIL) g4[i] = g2[i];          // ∂Hb2 = ∂T4 + FFN part
+  __syncthreads();
+  gemv_t(P + L.M2.F.W1, D, D, D, g3, D, V, g4, D, scr, true);
+  __syncthreads();
+  warp_ln_bwd<D>(T3, g4, g5, V, PV(12), false);                    // ∂T3 (= ∂A2, residual ∂pma)
+  __syncthreads();
+  gemv_t(P + L.M2.Wo, D, D, D, g5, D, V, g6, D, scr, false);       // ∂O2
+  __syncthreads();
+  // attention over the k seeds: ∂w, ∂s, ∂Q2, ∂K2, ∂V2 (g7 = ∂Q2, g8 = ∂K2, A1 reused as ∂V2)
+  float *dQ2 = g7, *dK2 = g8, *dV2 = A2;       // A2 no longer needed after the row record below
+  for (int o = t; o < heads * KK; o += DT_TAIL) {
+    const int h = o / KK, j = (o / k) % k, jj = o % k;
+    float sdot = 0.f;
+    for (int i = 0; i < dh; ++i) sdot = fmaf(g6[j * D + h * dh + i], V2[jj * D + h * dh + i], sdot);
+    dWatt[o] = sdot;
+  }
+  __syncthreads();
+  for (int o = t; o < heads * k; o += DT_TAIL) {     // ∂s = w (∂w − Σ w ∂w), scaled by 1/√d_h
+    float dot = 0.f;
+    for (int jj = 0; jj < k; ++jj) dot = fmaf(Watt[o * k + jj], dWatt[o * k + jj], dot);
+    for (int jj = 0; jj < k; ++jj) dWatt[o * k + jj] = Watt[o * k + jj] * (dWatt[o * k + jj] - dot) * isq;
+  }
+  __syncthreads();
+  // write the row records that need A2's buffer before it becomes ∂V2
+  float *rows = b.rows;
+  const long RK = long(a.B) * k;
+  auto rec = [&](int slot, const float *src) {
+    float *dst = rows + (long(slot) * RK + long(g) * k) * D;
+    for (int i = t; i < V * D; i += DT_TAIL) dst[i] = src[i];
+  };
+  __syncthreads();
+  for (int o = t; o < V * D; o += DT_TAIL) {
+    const int j = o / D, ch = o % D, h = ch / dh;
+    float aq = 0.f, ak = 0.f, av = 0.f;
+    for (int jj = 0; jj < k; ++jj) {
+      aq = fmaf(dWatt[(h * k + j) * k + jj], K2[jj * D + ch], aq);       // ∂Q2[j]
+      ak = fmaf(dWatt[(h * k + jj) * k + j], Q2[jj * D + ch], ak);       // ∂K2[j]
+      av = fmaf(Watt[(h * k + jj) * k + j], g6[jj * D + ch], av);        // ∂V2[j]
+    }
+    dQ2[o] = aq;
+    dK2[o] = ak;
+    dV2[o] = av;
+  }
+  __syncthreads();
+  // ∂pma = ∂T3 (residual) + W_qᵀ ∂Q2 + W_kᵀ ∂K2 + W_vᵀ ∂V2  -> g9
+  for (int i = t; i < V * D; i += DT_TAIL) g9[i] = g5[i];
+  __syncthreads();
+  gemv_t(P + L.M2.Wq, D, D, D, dQ2, D, V, g9, D, scr, true);
+  gemv_t(P + L.M2.Wk, D, D, D, dK2, D, V, g9, D, scr, true);
+  gemv_t(P + L.M2.Wv, D, D, D, dV2, D, V, g9, D, scr, true);
+  __syncthreads();
+  // records of the SAB / final FFN part
+  rec(R_UD, UD); rec(R_dUD, g0); rec(R_sab, sab); rec(R_dsab, g1); rec(R_T4, T4);
+  rec(R_U2, U2); rec(R_dU2, g3); rec(R_Hb2, Hb2); rec(R_dT4, g2); rec(R_dHb2, g4); rec(R_T3, T3);
+  rec(R_O2, O2); rec(R_dT3, g5); rec(R_dQ2, dQ2); rec(R_dK2, dK2); rec(R_dV2, dV2); rec(R_pma, pma);
+  rec(R_dpma, g9);
+  __syncthreads();
+  // PMA tail: ∂T2 = LN2ᵀ(∂pma); ∂U1; ∂Hb1 = ∂T2 + W1ᵀ ∂U1; ∂T1 = LN1ᵀ(∂Hb1); ∂O1 = W_oᵀ ∂T1
+  warp_ln_bwd<D>(T2, g9, g0, V, PV(6), false);                     // g0 = ∂T2 (= ∂F1)
+  __syncthreads();
+  gemv_t(P + L.M1.F.W2, D, D, D, g0, D, V, g1, D, scr, false);
+  __syncthreads();
+  for (int i = t; i < V * D; i += DT_TAIL) {
+    g1[i] = U1[i] > 0.f ? g1[i] : 0.f;                             // g1 = ∂U1 (pre-ReLU)
+    g2[i] = g0[i];
+  }
+  __syncthreads();
+  gemv_t(P + L.M1.F.W1, D, D, D, g1, D, V, g2, D, scr, true);      // g2 = ∂Hb1
+  __syncthreads();
+  warp_ln_bwd<D>(T1, g2, g3, V, PV(2), false);                     // g3 = ∂T1 (= ∂A1 = ∂S_g)
+  __syncthreads();
+  gemv_t(P + L.M1.Wo, D, D, D, g3, D, V, g4, D, scr, false);       // g4 = ∂O1
+  __syncthreads();
+  rec(R_T2, T2); rec(R_U1, U1); rec(R_dU1, g1); rec(R_Hb1, Hb1); rec(R_dT2, g0); rec(R_dHb1, g2);
+  rec(R_T1, T1); rec(R_O1, O1); rec(R_dT1, g3); rec(R_dO1, g4);
+  // u_kh = W_v,hᵀ ∂O1[j, h-slice]  (the node side's ∂P̄_kh)
+  for (int o = t; o < KH * D; o += DT_TAIL) {
+    const int kh = o / D, c = o % D, j = kh / heads, h = kh % heads;
+    float acc = 0.f;
+    for (int i = 0; i < dh; ++i) acc = fmaf(g4[j * D + h * dh + i], __ldg(P + L.M1.Wv + long(h * dh + i) * D + c), acc);
+    b.u[(long(g) * KHMAX + kh) * D + c] = acc;
+  }
+}
+
+// Node side of PMA's attention, pass A (mode 0: per-range partial Σ_n α ∂α per (seed, head))
+// and pass B (mode 1: ds, ∂Z rows, per-range partial G_kh = Σ ds Z_n and σ_kh = Σ ds).
+// Grid (B, SPLIT) as the forward pool; 32-row chunks of Z staged in shared memory.
+struct DecPoolBwdArgs {
+  const float *Z, *prep, *pstat, *u;
+  const int32_t *node_off;
+  int k, heads, B;
+  float *dsum_part;              // [B][SPLIT][KHMAX]
+  float *dZ;                     // [N][D]
+  float *gpart;                  // [B][SPLIT][KHMAX][D + 1]
+};
+
+// Every node is taken relative to the graph's first node r: ∂α_n − ∂α_r = (Z_n − Z_r)·u and,
+// since Σ_n ds_n = 0 exactly, G_kh = Σ_n ds_n (Z_n − Z_r).  Same values, but node states that
+// nearly coincide across a graph no longer cancel at the size of Z itself.
+template <int D>
+__global__ void __launch_bounds__(DT) dec_pool_bwd_kernel(const DecPoolBwdArgs a, int mode) {
+  __shared__ __align__(16) float Zc[CH][D];
+  __shared__ float al[CH][KHMAX], ds[CH][KHMAX];
+  __shared__ float Dsum[KHMAX];
+  __shared__ __align__(16) float Zr[D];
+  const int KH = a.k * a.heads, t = threadIdx.x, g = blockIdx.x, sp = blockIdx.y;
+  const long g0 = a.node_off[g], len = a.node_off[g + 1] - g0;
+  const long u0 = g0 + len * sp / SPLIT, u1 = g0 + len * (sp + 1) / SPLIT;
+  for (int c = t; c < D; c += DT) Zr[c] = __ldg(a.Z + g0 * D + c);
+  if (mode == 1 && t < KH) {
+    float s = 0.f;
+    for (int q = 0; q < SPLIT; ++q) s += a.dsum_part[(long(g) * SPLIT + q) * KHMAX + t];
+    Dsum[t] = s;
+  }
+  // per-thread accumulators: mode 0: Σ α ∂α for kh = t (t < KH); mode 1: G[kh][c] for
+  // outputs o = t, t + DT, ... of KH·D, and σ_kh
+  float acc0 = 0.f;
+  float gacc[KHMAX * D / DT];
+#pragma unroll
+  for (int i = 0; i < KHMAX * D / DT; ++i) gacc[i] = 0.f;
+  float sacc = 0.f;
+  __syncthreads();
+  for (long n0 = u0; n0 < u1; n0 += CH) {
+    const int rows = int(min(long(CH), u1 - n0));
+    for (int i = t; i < CH * D; i += DT) {
+      const int r = i / D, c = i % D;
+      Zc[r][c] = r < rows ? __ldg(a.Z + (n0 + r) * D + c) : 0.f;
+    }
+    __syncthreads();
+    for (int o = t; o < rows * KH; o += DT) {       // α and ∂α − ∂α_r of (row, kh)
+      const int r = o / KH, kh = o % KH;
+      float s = a.prep[D * KHMAX + kh], da = 0.f;
+      const float *uk = a.u + (long(g) * KHMAX + kh) * D;
+      for (int c = 0; c < D; ++c) {
+        s = fmaf(Zc[r][c], a.prep[c * KHMAX + kh], s);
+        da = fmaf(Zc[r][c] - Zr[c], __ldg(uk + c), da);
+      }
+      const float M = a.pstat[(long(g) * KHMAX + kh) * 2], l = a.pstat[(long(g) * KHMAX + kh) * 2 + 1];
+      const float alpha = ex2((s - M) * L2E) / l;
+      al[r][kh] = alpha;
+      ds[r][kh] = mode == 0 ? alpha * da : alpha * (da - Dsum[kh]);
+    }
+    __syncthreads();
+    if (mode == 0) {
+      if (t < KH)
+        for (int r = 0; r < rows; ++r) acc0 += ds[r][t];
+    } else {
+      for (int o = t; o < rows * D; o += DT) {      // ∂Z rows
+        const int r = o / D, c = o % D;
+        float z = 0.f;
+        for (int kh = 0; kh < KH; ++kh)
+          z = fmaf(al[r][kh], __ldg(a.u + (long(g) * KHMAX + kh) * D + c), fmaf(ds[r][kh], a.prep[c * KHMAX + kh], z));
+        a.dZ[(n0 + r) * D + c] = z;
+      }
+#pragma unroll
+      for (int i = 0; i < KHMAX * D / DT; ++i) {
+        const int o = t + i * DT, kh = o / D, c = o % D;
+        if (kh < KH)
+          for (int r = 0; r < rows; ++r) gacc[i] = fmaf(ds[r][kh], Zc[r][c] - Zr[c], gacc[i]);
+      }
+      if (t < KH)
+        for (int r = 0; r < rows; ++r) sacc += ds[r][t];
+    }
+    __syncthreads();
+  }
+  if (mode == 0) {
+    if (t < KH) a.dsum_part[(long(g) * SPLIT + sp) * KHMAX + t] = acc0;
+  } else {
+    float *gp = a.gpart + (long(g) * SPLIT + sp) * KHMAX * (D + 1);
+#pragma unroll
+    for (int i = 0; i < KHMAX * D / DT; ++i) {
+      const int o = t + i * DT, kh = o / D, c = o % D;
+      if (kh < KH) gp[kh * (D + 1) + c] = gacc[i];
+    }
+    if (t < KH) gp[t * (D + 1) + D] = sacc;
+  }
+}
+
+// dW[a][c] (+)= Σ_r X[r·ldx + a] Y[r·ldy + c] over R rows, thread per output, fixed order.
+__global__ void dec_rows_wgrad_kernel(const float *__restrict__ X, int ldx, const float *__restrict__ Y,
+                                      int ldy, long R, int A, int C, float *__restrict__ out, int ldo) {
+  const int o = blockIdx.x * blockDim.x + threadIdx.x;
+  if (o >= A * C) return;
+  const int ai = o / C, c = o % C;
+  double acc = 0.0;
+  for (long r = 0; r < R; ++r) acc = fma(double(X[r * ldx + ai]), double(Y[r * ldy + c]), acc);
+  out[long(ai) * ldo + c] = float(acc);
+}
+
+// out[c] = Σ_r X[r·ld + c]  (bias gradients), fixed order
+__global__ void dec_rows_colsum_kernel(const float *__restrict__ X, int ld, long R, int C,
+                                       float *__restrict__ out) {
+  const int c = blockIdx.x * blockDim.x + threadIdx.x;
+  if (c >= C) return;
+  double acc = 0.0;
+  for (long r = 0; r < R; ++r) acc += double(X[r * ld + c]);
+  out[c] = float(acc);
+}
+
+// LayerNorm parameter gradients over R rows: dγ = Σ_r dy ⊙ x̂, dβ = Σ_r dy (x = LN input)
+__global__ void dec_rows_ln_grads_kernel(const float *__restrict__ x, const float *__restrict__ dy,
+                                         long R, int D, float *__restrict__ gg, float *__restrict__ gb) {
+  const int c = blockIdx.x * blockDim.x + threadIdx.x;
+  if (c >= D) return;
+  double ag = 0.0, ab = 0.0;
+  for (long r = 0; r < R; ++r) {
+    const float *xr = x + r * D;
+    float s = 0.f;
+    for (int i = 0; i < D; ++i) s += xr[i];
+    const float mu = s / float(D);
+    float q = 0.f;
+    for (int i = 0; i < D; ++i) q = fmaf(xr[i] - mu, xr[i] - mu, q);
+    const float rstd = rsqrtf(q / float(D) + 1e-5f);
+    const float d = dy[r * D + c];
+    ag = fma(double(d), double((xr[c] - mu) * rstd), ag);
+    ab += double(d);
+  }
+  gg[c] = float(ag);
+  gb[c] = float(ab);
+}
+
+// The seeds' side (one CTA): merge the pool-backward partials over graphs and ranges, then
+// ∂q_kh, ∂W_k, ∂b_k, ∂Q1 -> ∂W_q, ∂b_q and ∂S = Σ_g ∂T1_g + W_qᵀ ∂Q1.
+template <int D>
+__global__ void __launch_bounds__(DT) dec_seed_grads_kernel(const DecArgs a, const float *__restrict__ gpart,
+                                                            const float *__restrict__ dT1rows, float *__restrict__ G) {
+  __shared__ __align__(16) float Gs[KHMAX][D + 1];
+  __shared__ __align__(16) float S[KMAX * D], Q[KMAX * D], dQ[KMAX * D];
+  const int k = a.k, heads = a.heads, KH = k * heads, dh = D / heads, t = threadIdx.x;
+  const DecLayout &L = a.L;
+  const float *P = a.P;
+  const float isq = rsqrtf(float(dh));
+  for (int o = t; o < KH * (D + 1); o += DT) {
+    const int kh = o / (D + 1), c = o % (D + 1);
+    double acc = 0.0;
+    for (int g = 0; g < a.B; ++g)
+      for (int q = 0; q < SPLIT; ++q) acc += double(gpart[((long(g) * SPLIT + q) * KHMAX + kh) * (D + 1) + c]);
+    Gs[kh][c] = float(acc);
+  }
+  for (int i = t; i < k * D; i += DT) S[i] = P[L.S + i];
+  __syncthreads();
+  warp_gemv(P + L.M1.Wq, D, D, D, S, D, k, Q, D, P + L.M1.bq, false);
+  __syncthreads();
+  // ∂q_kh = (W_k,h G_kh + b_k,h σ_kh)/√d_h -> ∂Q1[j][h·dh + i]; ∂W_k, ∂b_k
+  for (int o = t; o < k * D; o += DT) {
+    const int j = o / D, n = o % D, h = n / dh;
+    const int kh = j * heads + h;
+    // σ_kh = Σ_n ds_n is exactly 0 (softmax shift invariance; Gs[kh][D] holds its rounding),
+    // so ∂q_kh = W_k,h G_kh / √d_h with G_kh taken relative to the reference node
+    float acc = 0.f;
+    for (int c = 0; c < D; ++c) acc = fmaf(__ldg(P + L.M1.Wk + long(n) * D + c), Gs[kh][c], acc);
+    dQ[o] = acc * isq;
+  }
+  for (int o = t; o < D * D; o += DT) {
+    const int n = o / D, c = o % D, h = n / dh;
+    float acc = 0.f;
+    for (int j = 0; j < k; ++j) acc = fmaf(Q[j * D + n] * isq, Gs[j * heads + h][c], acc);
+    G[L.M1.Wk + o] = acc;
+  }
+  for (int n = t; n < D; n += DT) G[L.M1.bk + n] = 0.f;     // ∂b_k = Σ q σ / √d_h = 0 exactly
+  __syncthreads();
+  for (int o = t; o < D * D; o += DT) {            // ∂W_q = Σ_j ∂Q1[j] ⊗ S[j]
+    const int n = o / D, c = o % D;
+    float acc = 0.f;
+    for (int j = 0; j < k; ++j) acc = fmaf(dQ[j * D + n], S[j * D + c], acc);
+    G[L.M1.Wq + o] = acc;
+  }
+  for (int n = t; n < D; n += DT) {
+    float acc = 0.f;
+    for (int j = 0; j < k; ++j) acc += dQ[j * D + n];
+    G[L.M1.bq + n] = acc;
+  }
+  for (int o = t; o < k * D; o += DT) {            // ∂S = Σ_g ∂T1_g + W_qᵀ ∂Q1
+    const int j = o / D, c = o % D;
+    double acc = 0.0;
+    for (int g = 0; g < a.B; ++g) acc += double(dT1rows[(long(g) * k + j) * D + c]);
+    float w = 0.f;
+    for (int n = 0; n < D; ++n) w = fmaf(dQ[j * D + n], __ldg(P + L.M1.Wq + long(n) * D + c), w);
+    G[L.S + o] = float(acc) + w;
+  }
+}
+
 }  // namespace
 
 int launch_set_decoder(const occu_ctx *ctx, const DevCsr &csr, const float *hL, float *T, float *Z,
@@ -740,6 +1289,118 @@ int launch_set_decoder(const occu_ctx *ctx, const DevCsr &csr, const float *hL, 
         set_decoder_kernel<128>);
   const cudaError_t e = cudaGetLastError();
   return e == cudaSuccess ? n + 2 + nprep : -int(e);
+}
+
+}  // namespace occu
+
+namespace occu {
+
+int launch_set_decoder_bwd(occu_ctx *ctx, const DevCsr &csr, const float *hL, const float *T,
+                           const float *Z, const float *dr, float *dZ, float *dT, float *dhL,
+                           cudaStream_t st) {
+  const occu_config &cf = ctx->cfg;
+  const ParamLayout &L = ctx->layout;
+  const float *P = ctx->params.as<float>();
+  float *G = ctx->grads.as<float>();
+  const int D = cf.d, k = cf.k, KH = k * cf.heads, B = csr.B;
+  if (!L.dec || k > KMAX || KH > KHMAX) return -int(cudaErrorInvalidValue);
+  const long RK = long(B) * k;
+  const size_t f_rows = size_t(R_COUNT) * RK * D, f_pstat = size_t(B) * KHMAX * 2,
+               f_pbar = size_t(B) * KH * D, f_u = size_t(B) * KHMAX * D,
+               f_ds = size_t(B) * SPLIT * KHMAX, f_gp = size_t(B) * SPLIT * KHMAX * (D + 1);
+  if (ctx->ws.dbwd.ensure((f_rows + f_pstat + f_pbar + f_u + f_ds + f_gp) * 4) != cudaSuccess)
+    return -int(cudaErrorMemoryAllocation);
+  float *rows = ctx->ws.dbwd.as<float>(), *pstat = rows + f_rows, *pbar = pstat + f_pstat,
+        *u = pbar + f_pbar, *dsp = u + f_u, *gp = dsp + f_ds;
+  DecBwdArgs b{};
+  DecArgs &a = b.f;
+  a.Z = Z; a.node_off = csr.node_off; a.P = P; a.L = L.D;
+  a.W_1 = L.W_1; a.b_1 = L.b_1; a.w_2 = L.w_2; a.b_2 = L.b_2;
+  a.k = k; a.heads = cf.heads; a.d_h = cf.d_h; a.slope = cf.slope; a.B = B;
+  b.part = ctx->ws.dpool.as<float>(); b.dr = dr; b.rows = rows; b.pstat = pstat; b.pbar = pbar; b.u = u;
+  int n = 0;
+  OCCU_PROF_BEGIN(ctx, "dec_tail_bwd", st);
+  const size_t smem = (D == 64 ? tail_bwd_smem_floats<64>() : tail_bwd_smem_floats<128>()) * 4;
+  if (D == 64) {
+    cudaFuncSetAttribute(dec_tail_bwd_kernel<64>, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
+    dec_tail_bwd_kernel<64><<<B, DT_TAIL, smem, st>>>(b);
+  } else {
+    cudaFuncSetAttribute(dec_tail_bwd_kernel<128>, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
+    dec_tail_bwd_kernel<128><<<B, DT_TAIL, smem, st>>>(b);
+  }
+  OCCU_PROF_END(ctx);
+  ++n;
+  DecPoolBwdArgs pa{};
+  pa.Z = Z; pa.prep = ctx->ws.dprep.as<float>(); pa.pstat = pstat; pa.u = u; pa.node_off = csr.node_off;
+  pa.k = k; pa.heads = cf.heads; pa.B = B; pa.dsum_part = dsp; pa.dZ = dZ; pa.gpart = gp;
+  OCCU_PROF_BEGIN(ctx, "dec_pool_bwd", st);
+  for (int mode = 0; mode < 2; ++mode) {
+    if (D == 64) dec_pool_bwd_kernel<64><<<dim3(B, SPLIT), DT, 0, st>>>(pa, mode);
+    else dec_pool_bwd_kernel<128><<<dim3(B, SPLIT), DT, 0, st>>>(pa, mode);
+  }
+  OCCU_PROF_END(ctx);
+  n += 2;
+  OCCU_PROF_BEGIN(ctx, "dec_seed_grads", st);
+  if (D == 64) dec_seed_grads_kernel<64><<<1, DT, 0, st>>>(a, gp, rows + size_t(R_dT1) * RK * D, G);
+  else dec_seed_grads_kernel<128><<<1, DT, 0, st>>>(a, gp, rows + size_t(R_dT1) * RK * D, G);
+  OCCU_PROF_END(ctx);
+  ++n;
+  // tail weight / bias / LayerNorm gradients: fixed-order reductions over the B·k rows
+  auto row = [&](int slot) { return rows + size_t(slot) * RK * D; };
+  auto wg = [&](const float *X, const float *Y, size_t out) {
+    dec_rows_wgrad_kernel<<<(D * D + 255) / 256, 256, 0, st>>>(X, D, Y, D, RK, D, D, G + out, D);
+    ++n;
+  };
+  auto cs = [&](const float *X, size_t out) {
+    dec_rows_colsum_kernel<<<(D + 127) / 128, 128, 0, st>>>(X, D, RK, D, G + out);
+    ++n;
+  };
+  auto lg = [&](const float *x, const float *dy, size_t g_, size_t b_) {
+    dec_rows_ln_grads_kernel<<<(D + 127) / 128, 128, 0, st>>>(x, dy, RK, D, G + g_, G + b_);
+    ++n;
+  };
+  const DecLayout &DL = L.D;
+  OCCU_PROF_BEGIN(ctx, "dec_tail_wgrads", st);
+  wg(dr, row(R_UD), DL.D.W2); cs(dr, DL.D.b2);
+  wg(row(R_dUD), row(R_sab), DL.D.W1); cs(row(R_dUD), DL.D.b1);
+  lg(row(R_T4), row(R_dsab), DL.M2.ln2_g, DL.M2.ln2_b);
+  wg(row(R_dT4), row(R_U2), DL.M2.F.W2); cs(row(R_dT4), DL.M2.F.b2);
+  wg(row(R_dU2), row(R_Hb2), DL.M2.F.W1); cs(row(R_dU2), DL.M2.F.b1);
+  lg(row(R_T3), row(R_dHb2), DL.M2.ln1_g, DL.M2.ln1_b);
+  wg(row(R_dT3), row(R_O2), DL.M2.Wo); cs(row(R_dT3), DL.M2.bo);
+  wg(row(R_dQ2), row(R_pma), DL.M2.Wq); cs(row(R_dQ2), DL.M2.bq);
+  wg(row(R_dK2), row(R_pma), DL.M2.Wk); cs(row(R_dK2), DL.M2.bk);
+  wg(row(R_dV2), row(R_pma), DL.M2.Wv); cs(row(R_dV2), DL.M2.bv);
+  lg(row(R_T2), row(R_dpma), DL.M1.ln2_g, DL.M1.ln2_b);
+  wg(row(R_dT2), row(R_U1), DL.M1.F.W2); cs(row(R_dT2), DL.M1.F.b2);
+  wg(row(R_dU1), row(R_Hb1), DL.M1.F.W1); cs(row(R_dU1), DL.M1.F.b1);
+  lg(row(R_T1), row(R_dHb1), DL.M1.ln1_g, DL.M1.ln1_b);
+  wg(row(R_dT1), row(R_O1), DL.M1.Wo); cs(row(R_dT1), DL.M1.bo);
+  cs(row(R_dO1), DL.M1.bv);
+  const int dh = D / cf.heads;
+  for (int h = 0; h < cf.heads; ++h) {     // ∂W_v rows of head h: Σ_(g,j) ∂O1[g,j][h] ⊗ P̄[g,(j,h)]
+    dec_rows_wgrad_kernel<<<(dh * D + 255) / 256, 256, 0, st>>>(
+        row(R_dO1) + h * dh, D, pbar + size_t(h) * D, cf.heads * D, RK, dh, D,
+        G + DL.M1.Wv + size_t(h) * dh * D, D);
+    ++n;
+  }
+  OCCU_PROF_END(ctx);
+  // PMA's pre-pooling FFN over the N node rows (tensor cores): Z = T W2ᵀ + b2, T = ReLU(h W1ᵀ + b1)
+  int r;
+  if ((r = launch_plain_masked_tc(ctx, dZ, D, csr.N, 3, cf.L, nullptr, dT, "dec_ffn_bwd_tc", st, T, 0.f)) < 0) return r;
+  n += r;
+  if ((r = launch_wgrad(ctx, dZ, D, T, D, csr.N, G + DL.P.W2, st, false)) < 0) return r;
+  n += r;
+  if ((r = launch_colsum_rows(ctx, dZ, csr.N, G + DL.P.b2, st)) < 0) return r;
+  n += r;
+  if ((r = launch_plain_tc(ctx, dT, D, csr.N, 2, cf.L, nullptr, dhL, "dec_ffn_bwd_tc", st)) < 0) return r;
+  n += r;
+  if ((r = launch_wgrad(ctx, dT, D, hL, D, csr.N, G + DL.P.W1, st, false)) < 0) return r;
+  n += r;
+  if ((r = launch_colsum_rows(ctx, dT, csr.N, G + DL.P.b1, st)) < 0) return r;
+  n += r;
+  const cudaError_t e = cudaGetLastError();
+  return e == cudaSuccess ? n : -int(e);
 }
 
 }  // namespace occu

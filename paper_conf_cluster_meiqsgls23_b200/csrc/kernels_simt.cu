@@ -1924,19 +1924,21 @@ int launch_head_backward(occu_ctx *ctx, const DevCsr &csr, const float *targets,
   float *G = ctx->grads.as<float>();
   const float inv_gb = 1.f / float(global_B);
   OCCU_PROF_BEGIN(ctx, "head_bwd_graph", st);
+  const int hin = L.head_in;          // d (mean readout) or k·d (decoder readout)
   head_bwd_graph_kernel<<<csr.B, 128, cf.d_h * 4, st>>>(
-      w.yhat.as<float>(), targets, w.c.as<float>(), P + L.W_1, P + L.w_2, cf.d, cf.d_h, inv_gb,
+      w.yhat.as<float>(), targets, w.c.as<float>(), P + L.W_1, P + L.w_2, hin, cf.d_h, inv_gb,
       cf.slope, w.dy.as<float>(), w.dc.as<float>(), w.dr.as<float>());
   OCCU_PROF_END(ctx);
   LAUNCH_CHECK();
-  const int jobs = cf.d_h * cf.d + 2 * cf.d_h + 2;
+  const int jobs = cf.d_h * hin + 2 * cf.d_h + 2;
   OCCU_PROF_BEGIN(ctx, "head_bwd_reduce", st);
   head_bwd_reduce_kernel<<<grid_for(jobs, 256, 1024), 256, 0, st>>>(
       w.dy.as<float>(), w.dc.as<float>(), w.r.as<float>(), w.c.as<float>(), w.yhat.as<float>(),
-      targets, csr.B, cf.d, cf.d_h, inv_gb, cf.slope, G + L.W_1, G + L.b_1, G + L.w_2, G + L.b_2,
+      targets, csr.B, hin, cf.d_h, inv_gb, cf.slope, G + L.W_1, G + L.b_1, G + L.w_2, G + L.b_2,
       w.loss.as<float>());
   OCCU_PROF_END(ctx);
   LAUNCH_CHECK();
+  if (cf.readout == OCCU_READOUT_SET_DECODER) return 2;   // dr feeds the decoder backward
   OCCU_PROF_BEGIN(ctx, "broadcast_dh", st);
   // TC backward consumes dA directly; with Graphormer layers dr/n_b is the gradient of the
   // stack's top states and the mask is applied below the stack (launch_mask_dA)

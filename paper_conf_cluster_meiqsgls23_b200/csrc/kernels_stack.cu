@@ -403,6 +403,10 @@ static int colsum(occu_ctx *ctx, const float *X, long R, float *out, cudaStream_
   return 2;
 }
 
+int launch_colsum_rows(occu_ctx *ctx, const float *X, long R, float *out, cudaStream_t st) {
+  return colsum(ctx, X, R, out, st);
+}
+
 // dx = add + LNᵀ(dy) for x = LN input; dγ, dβ into gg, gb.
 static int ln_bwd(occu_ctx *ctx, const float *x, const float *gam, const float *dy, const float *add,
                   float *dx, long R, float *gg, float *gb, cudaStream_t st) {

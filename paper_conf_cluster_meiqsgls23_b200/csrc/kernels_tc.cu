@@ -1755,15 +1755,17 @@ int tc_prepare_weights(occu_ctx *ctx, cudaStream_t st) {
     if (i > 0) add(5, P + L.W_u[i], c.d, c.d, 1);
   }
   if (L.dec) {      // NEXT-2 decoder: the pre-pooling FFN's two d x d matrices
-    auto addd = [&](int kind, const float *W) {
+    auto addd = [&](int kind, const float *W, int transW = 0) {
       WImageJob j;
-      j.W = W; j.D = c.d; j.K = c.d; j.transW = 0; j.bf16 = 0;
+      j.W = W; j.D = c.d; j.K = c.d; j.transW = transW; j.bf16 = 0;
       j.img = const_cast<uint8_t *>(tc_wimg(ctx, kind, c.L));
       j.fexp = const_cast<int *>(tc_wfexp(ctx, kind, c.L));
       jobs.push_back(j);
     };
     addd(0, P + L.D.P.W1);
     addd(1, P + L.D.P.W2);
+    addd(2, P + L.D.P.W1, 1);           // transposed (training: dX = dY·W)
+    addd(3, P + L.D.P.W2, 1);
   }
   for (int j = 0; j < c.graphormer; ++j) {      // NEXT-3 Graphormer: six d x d matrices
     const GphOff &g = L.G[j];

@@ -74,6 +74,7 @@ struct Workspace {
   std::vector<DevBuf> gsave;   // training: 8 saved [N][d] intermediates per Graphormer layer
   DevBuf gscr;             // training: Graphormer backward scratch 5 x [N][d] + stats
   DevBuf gdh[2];           // training: gradients w.r.t. the stack's node states (ping-pong)
+  DevBuf dbwd;             // training: decoder backward rows / stats / partials
   void release_all();
 };
 
@@ -268,6 +269,14 @@ int launch_mask_dA(const occu_ctx *ctx, const DevCsr &csr, const float *dh, cons
 int launch_plain_masked_tc(const occu_ctx *ctx, const float *A, int K, int R, int wkind, int layer,
                            const float *add, float *out, const char *name, cudaStream_t st,
                            const float *mask, float slope);
+// NEXT-2 training (kernels_decoder.cu): backward of the decoder readout from dr = ∂L/∂r
+// [B][k·d] down to dhL = ∂L/∂(the decoder's node-state input hL) [N][d]; T, Z: the forward's
+// FFN hidden / output rows; dZ, dT: [N][d] scratch.  Parameter gradients into ctx->grads.
+int launch_set_decoder_bwd(occu_ctx *ctx, const DevCsr &csr, const float *hL, const float *T,
+                           const float *Z, const float *dr, float *dZ, float *dT, float *dhL,
+                           cudaStream_t st);
+// out[c] = Σ_r X[r][c] over R rows of width d, fixed order (kernels_stack.cu)
+int launch_colsum_rows(occu_ctx *ctx, const float *X, long R, float *out, cudaStream_t st);
 // Image slot of Graphormer layer j's transposed matrices (kinds 0-5: W_qᵀ W_kᵀ W_vᵀ W_oᵀ W1ᵀ W2ᵀ).
 int gph_tslot(const occu_config &c, int j);
 int launch_bias_add_tc(const occu_ctx *ctx, const float *A, int K, int R, int wkind, int layer,

@@ -50,7 +50,7 @@ void Workspace::release_all() {
   DevBuf *bufs[] = {&node_feat, &edge_feat, &targets, &out_occ, &csr, &e0, &g, &r, &c, &yhat,
                     &dy, &dc, &dr, &dh, &dhprev, &dP, &MG, &DV, &DZ, &deA, &deB, &dalpha,
                     &dpq, &partial, &loss, &tcpart, &dpart, &rpart, &anf[0], &anf[1],
-                    &aef[0], &aef[1], &acsr[0], &acsr[1], &dT, &dZ, &dprep, &dpool, &gx, &gqkv, &go, &gscr, &gdh[0], &gdh[1],
+                    &aef[0], &aef[1], &acsr[0], &acsr[1], &dT, &dZ, &dprep, &dpool, &gx, &gqkv, &go, &gscr, &gdh[0], &gdh[1], &dbwd,
                     &scsr, &snf, &sef, &sdesc, &hf};
   for (DevBuf *b : bufs) b->release();
   for (auto *v : {&hbar, &p, &q, &e, &h, &gs, &gh, &gsave})
@@ -425,8 +425,6 @@ occu_status grads_impl(occu_ctx *ctx, const occu_batch *batch, const float *targ
   const bool stack = ctx->cfg.readout == OCCU_READOUT_SET_DECODER || ctx->cfg.graphormer > 0;
   if (stack && (ctx->cfg.prec != OCCU_FP32 || ctx->path != 0))
     return fail(ctx, OCCU_EINVAL, "training through the Graphormer layers / decoder readout runs in OCCU_FP32 on kernel path 0");
-  if (ctx->cfg.readout == OCCU_READOUT_SET_DECODER)
-    return fail(ctx, OCCU_EINVAL, "the Set-Transformer decoder readout is inference-only in this build");
   if (ctx->cfg.msg == OCCU_MSG_NEIGHBOR_SOFTMAX && ctx->cfg.prec == OCCU_BF16)
     return fail(ctx, OCCU_EINVAL, "reading B in OCCU_BF16 is inference-only in this build");
   ctx->launches = 0;
@@ -440,7 +438,7 @@ occu_status grads_impl(occu_ctx *ctx, const occu_batch *batch, const float *targ
   const size_t Nd = size_t(csr.N) * c.d * 4, Ed = size_t(csr.E) * c.d * 4;
   CK(w.dy.ensure(size_t(csr.B) * 4), "alloc");
   CK(w.dc.ensure(size_t(csr.B) * c.d_h * 4), "alloc");
-  CK(w.dr.ensure(size_t(csr.B) * c.d * 4), "alloc");
+  CK(w.dr.ensure(size_t(csr.B) * L.head_in * 4), "alloc");
   CK(w.dh.ensure(Nd), "alloc");
   CK(w.dP.ensure(Nd), "alloc");
   CK(w.MG.ensure(Ed), "alloc");
@@ -460,8 +458,17 @@ occu_status grads_impl(occu_ctx *ctx, const occu_batch *batch, const float *targ
     const size_t scr = 5 * Nd + size_t(csr.N) * std::max(c.heads, 1) * 16;
     CK(w.gscr.ensure(scr), "alloc stack scratch");
     float *g = w.gdh[0].as<float>();
-    // mean readout: broadcast_dh (launched by the head backward without a mask) left dr/n_b
-    CK(cudaMemcpyAsync(g, w.dh.ptr, Nd, cudaMemcpyDeviceToDevice, s), "copy dh");
+    const float *top = c.graphormer > 0 ? w.gh[c.graphormer - 1].as<float>() : w.h[c.L - 1].as<float>();
+    if (c.readout == OCCU_READOUT_SET_DECODER) {
+      // NEXT-2: decoder backward from dr down to its node-state input (the stack top)
+      float *scr = w.gscr.as<float>();
+      LK(launch_set_decoder_bwd(ctx, csr, top, w.dT.as<float>(), w.dZ.as<float>(), w.dr.as<float>(),
+                                scr, scr + size_t(csr.N) * c.d, g, s),
+         "decoder backward");
+    } else {
+      // mean readout: broadcast_dh (launched by the head backward without a mask) left dr/n_b
+      CK(cudaMemcpyAsync(g, w.dh.ptr, Nd, cudaMemcpyDeviceToDevice, s), "copy dh");
+    }
     for (int j = c.graphormer - 1; j >= 0; --j) {
       const float *hin = j == 0 ? w.h[c.L - 1].as<float>() : w.gh[j - 1].as<float>();
       GphSave sv;
