@@ -43,7 +43,7 @@ import numpy as np  # noqa: E402
 L2_BYTES = 126 * 1024 * 1024
 LR = 1e-4                      # P273: Adam, lr = 1e-4
 ALL_SECTIONS = ["cfg3_bf16", "cfg2", "cfg2_train", "micro", "readingb", "decoder", "graphormer",
-                "paper_stack", "cfg1", "cfg4", "cfg5"]
+                "paper_stack", "paper_stack_train", "cfg1", "cfg4", "cfg5"]
 METRIC = "GNN graphs/sec (train & infer) at 1/2/4/8 B200; aggregation HBM GB/s vs peak"
 
 
@@ -742,6 +742,28 @@ class Bench:
                      {"ms_per_step": ms, "gpu_launches": launches,
                       "what": "ANEE x3 -> Graphormer x2 -> Set-Transformer decoder (k=4) -> head"})
             del m, csr
+
+    def sec_paper_stack_train(self):
+        """Training the paper's full model (P273: ANEE -> 2 Graphormer layers -> Set-Transformer
+        decoder -> head, Adam) on CFG2, FP32: forward with saves, MSE, backward through the
+        decoder, the Graphormer layers and the ANEE rounds, Adam."""
+        occu, torch = self.occu, self.torch
+        b = self._cfg2()
+        _, nf, ef, yt = self.cfg2_dev
+        B = b.num_graphs
+        gB = B * self.world
+        m = self.model(graphormer=2, heads=4, readout=occu.READOUT_SET_DECODER, k=4)
+        m.init_weights(42)
+        self.dist_init(m)
+        csr = m.to_device(self.cfg2_host_csr)
+        st = lambda: m.train_step(csr, nf, ef, yt, LR, global_num_graphs=gB, want_loss=False)
+        l0 = m.train_step(csr, nf, ef, yt, LR, global_num_graphs=gB)
+        ms, launches, prof, _ = self.measure(st, m)
+        self.put("cfg2_paper_stack_train_f32", gB / (ms * 1e-3), "f32",
+                 {"ms_per_step": ms, "gpu_launches": launches, "loss_first": l0,
+                  "kernel_ms_per_step": {k_: v[0] / self.args.steps for k_, v in prof.items()},
+                  "what": "train step: ANEE x3 -> Graphormer x2 -> decoder (k=4) -> head, Adam"})
+        del m, csr
 
     def sec_cfg1(self):
         from occu_gen import configs
