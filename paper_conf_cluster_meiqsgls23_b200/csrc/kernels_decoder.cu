@@ -684,8 +684,8 @@ __global__ void __launch_bounds__(DT_TAIL) set_decoder_kernel(const DecArgs a, c
 //   FFN_D, SAB (= MAB2: LN2, FFN, LN1, W_o, the k x k attention per head, W_q/W_k/W_v),
 //   PMA's tail (MAB1: LN2, FFN, LN1, W_o)  ->  dO1 = ∂L/∂(W_v P̄ + b_v) per (seed, head).
 // Weight gradients need sums over graphs: each graph writes its (input, output-gradient) rows
-// to row arrays [B·k][d] and fixed-order row reductions (dec_rows_wgrad_kernel, column sums,
-// LayerNorm parameter sums) form them afterwards.  The node side (dec_pool_bwd_kernel) uses
+// to row arrays [B·k][d] and the backward's fixed-order split-K wgrad kernels, column sums and
+// LayerNorm parameter sums form them afterwards.  The node side (dec_pool_bwd_kernel) uses
 // the folded key map of the forward: score s_n = Z_n·M_kh + c_kh, α = softmax_n(s), so with
 // u_kh = W_v,hᵀ dO1_kh:  ∂α_n = Z_n·u_kh,  ds_n = α_n (∂α_n − Σ_m α_m ∂α_m),
 //   ∂Z_n = Σ_kh (α_n,kh u_kh + ds_n,kh M_kh),   G_kh = Σ_n ds_n,kh Z_n,  σ_kh = Σ_n ds_n,kh,
@@ -798,6 +798,7 @@ struct DecBwdArgs {
   float *pstat;                  // [B][KHMAX][2]: merged pool max, sum
   float *pbar;                   // [B·k·heads][D] merged pooled Z (P̄)
   float *u;                      // [B][KHMAX][D]: W_v,hᵀ dO1_kh
+  float *dO1h;                   // [heads][B·k][dh]: ∂O1 head-major
 };
 
 template <int D>
@@ -855,7 +856,9 @@ __global__ void __launch_bounds__(DT_TAIL) dec_tail_bwd_kernel(const DecBwdArgs 
     float acc = 0.f;
     for (int q = 0; q < SPLIT; ++q) acc = fmaf(pg[q * PS + o], fs[q * KHMAX + kh], acc);
     Pacc[o] = acc / lsum[kh];
-    b.pbar[long(g) * KH * D + o] = Pacc[o];
+    // head-major [heads][B·k][D] (row (g, j) of head h), contiguous per head for the W_v gradient
+    const int j = kh / heads, h = kh % heads;
+    b.pbar[(long(h) * a.B * k + long(g) * k + j) * D + o % D] = Pacc[o];
   }
   __syncthreads();
   // ---- forward recompute (set_decoder_kernel's chain), every intermediate kept
@@ -1017,6 +1020,10 @@ __global__ void __launch_bounds__(DT_TAIL) dec_tail_bwd_kernel(const DecBwdArgs 
   __syncthreads();
   rec(R_T2, T2); rec(R_U1, U1); rec(R_dU1, g1); rec(R_Hb1, Hb1); rec(R_dT2, g0); rec(R_dHb1, g2);
   rec(R_T1, T1); rec(R_O1, O1); rec(R_dT1, g3); rec(R_dO1, g4);
+  for (int i = t; i < V * D; i += DT_TAIL) {     // ∂O1 head-major [heads][B·k][dh] (W_v gradient)
+    const int j = i / D, ch = i % D, h = ch / dh;
+    b.dO1h[(long(h) * a.B * k + long(g) * k + j) * dh + ch % dh] = g4[i];
+  }
   // u_kh = W_v,hᵀ ∂O1[j, h-slice]  (the node side's ∂P̄_kh)
   for (int o = t; o < KH * D; o += DT_TAIL) {
     const int kh = o / D, c = o % D, j = kh / heads, h = kh % heads;
@@ -1118,49 +1125,6 @@ __global__ void __launch_bounds__(DT) dec_pool_bwd_kernel(const DecPoolBwdArgs a
     }
     if (t < KH) gp[t * (D + 1) + D] = sacc;
   }
-}
-
-// dW[a][c] (+)= Σ_r X[r·ldx + a] Y[r·ldy + c] over R rows, thread per output, fixed order.
-__global__ void dec_rows_wgrad_kernel(const float *__restrict__ X, int ldx, const float *__restrict__ Y,
-                                      int ldy, long R, int A, int C, float *__restrict__ out, int ldo) {
-  const int o = blockIdx.x * blockDim.x + threadIdx.x;
-  if (o >= A * C) return;
-  const int ai = o / C, c = o % C;
-  double acc = 0.0;
-  for (long r = 0; r < R; ++r) acc = fma(double(X[r * ldx + ai]), double(Y[r * ldy + c]), acc);
-  out[long(ai) * ldo + c] = float(acc);
-}
-
-// out[c] = Σ_r X[r·ld + c]  (bias gradients), fixed order
-__global__ void dec_rows_colsum_kernel(const float *__restrict__ X, int ld, long R, int C,
-                                       float *__restrict__ out) {
-  const int c = blockIdx.x * blockDim.x + threadIdx.x;
-  if (c >= C) return;
-  double acc = 0.0;
-  for (long r = 0; r < R; ++r) acc += double(X[r * ld + c]);
-  out[c] = float(acc);
-}
-
-// LayerNorm parameter gradients over R rows: dγ = Σ_r dy ⊙ x̂, dβ = Σ_r dy (x = LN input)
-__global__ void dec_rows_ln_grads_kernel(const float *__restrict__ x, const float *__restrict__ dy,
-                                         long R, int D, float *__restrict__ gg, float *__restrict__ gb) {
-  const int c = blockIdx.x * blockDim.x + threadIdx.x;
-  if (c >= D) return;
-  double ag = 0.0, ab = 0.0;
-  for (long r = 0; r < R; ++r) {
-    const float *xr = x + r * D;
-    float s = 0.f;
-    for (int i = 0; i < D; ++i) s += xr[i];
-    const float mu = s / float(D);
-    float q = 0.f;
-    for (int i = 0; i < D; ++i) q = fmaf(xr[i] - mu, xr[i] - mu, q);
-    const float rstd = rsqrtf(q / float(D) + 1e-5f);
-    const float d = dy[r * D + c];
-    ag = fma(double(d), double((xr[c] - mu) * rstd), ag);
-    ab += double(d);
-  }
-  gg[c] = float(ag);
-  gb[c] = float(ab);
 }
 
 // The seeds' side (one CTA): merge the pool-backward partials over graphs and ranges, then
@@ -1307,17 +1271,19 @@ int launch_set_decoder_bwd(occu_ctx *ctx, const DevCsr &csr, const float *hL, co
   const long RK = long(B) * k;
   const size_t f_rows = size_t(R_COUNT) * RK * D, f_pstat = size_t(B) * KHMAX * 2,
                f_pbar = size_t(B) * KH * D, f_u = size_t(B) * KHMAX * D,
-               f_ds = size_t(B) * SPLIT * KHMAX, f_gp = size_t(B) * SPLIT * KHMAX * (D + 1);
-  if (ctx->ws.dbwd.ensure((f_rows + f_pstat + f_pbar + f_u + f_ds + f_gp) * 4) != cudaSuccess)
+               f_ds = size_t(B) * SPLIT * KHMAX, f_gp = size_t(B) * SPLIT * KHMAX * (D + 1),
+               f_h = size_t(RK) * D, f_x = size_t(RK) * D;
+  if (ctx->ws.dbwd.ensure((f_rows + f_pstat + f_pbar + f_u + f_ds + f_gp + f_h + f_x) * 4) != cudaSuccess)
     return -int(cudaErrorMemoryAllocation);
   float *rows = ctx->ws.dbwd.as<float>(), *pstat = rows + f_rows, *pbar = pstat + f_pstat,
-        *u = pbar + f_pbar, *dsp = u + f_u, *gp = dsp + f_ds;
+        *u = pbar + f_pbar, *dsp = u + f_u, *gp = dsp + f_ds, *dO1h = gp + f_gp, *xscr = dO1h + f_h;
   DecBwdArgs b{};
   DecArgs &a = b.f;
   a.Z = Z; a.node_off = csr.node_off; a.P = P; a.L = L.D;
   a.W_1 = L.W_1; a.b_1 = L.b_1; a.w_2 = L.w_2; a.b_2 = L.b_2;
   a.k = k; a.heads = cf.heads; a.d_h = cf.d_h; a.slope = cf.slope; a.B = B;
   b.part = ctx->ws.dpool.as<float>(); b.dr = dr; b.rows = rows; b.pstat = pstat; b.pbar = pbar; b.u = u;
+  b.dO1h = dO1h;
   int n = 0;
   OCCU_PROF_BEGIN(ctx, "dec_tail_bwd", st);
   const size_t smem = (D == 64 ? tail_bwd_smem_floats<64>() : tail_bwd_smem_floats<128>()) * 4;
@@ -1347,46 +1313,44 @@ int launch_set_decoder_bwd(occu_ctx *ctx, const DevCsr &csr, const float *hL, co
   ++n;
   // tail weight / bias / LayerNorm gradients: fixed-order reductions over the B·k rows
   auto row = [&](int slot) { return rows + size_t(slot) * RK * D; };
+  // (the split-K wgrad kernels of the backward, parallel column sums and LayerNorm sums)
+  int rr;
   auto wg = [&](const float *X, const float *Y, size_t out) {
-    dec_rows_wgrad_kernel<<<(D * D + 255) / 256, 256, 0, st>>>(X, D, Y, D, RK, D, D, G + out, D);
-    ++n;
+    if ((rr = launch_wgrad(ctx, X, D, Y, D, RK, G + out, st, false)) >= 0) n += rr;
   };
   auto cs = [&](const float *X, size_t out) {
-    dec_rows_colsum_kernel<<<(D + 127) / 128, 128, 0, st>>>(X, D, RK, D, G + out);
-    ++n;
+    if ((rr = launch_colsum_rows(ctx, X, RK, G + out, st)) >= 0) n += rr;
   };
-  auto lg = [&](const float *x, const float *dy, size_t g_, size_t b_) {
-    dec_rows_ln_grads_kernel<<<(D + 127) / 128, 128, 0, st>>>(x, dy, RK, D, G + g_, G + b_);
-    ++n;
+  auto lg = [&](const float *x, size_t gam, const float *dy, size_t g_, size_t b_) {
+    if ((rr = launch_ln_param_grads(ctx, x, P + gam, dy, RK, xscr, G + g_, G + b_, st)) >= 0) n += rr;
   };
   const DecLayout &DL = L.D;
   OCCU_PROF_BEGIN(ctx, "dec_tail_wgrads", st);
   wg(dr, row(R_UD), DL.D.W2); cs(dr, DL.D.b2);
   wg(row(R_dUD), row(R_sab), DL.D.W1); cs(row(R_dUD), DL.D.b1);
-  lg(row(R_T4), row(R_dsab), DL.M2.ln2_g, DL.M2.ln2_b);
+  lg(row(R_T4), DL.M2.ln2_g, row(R_dsab), DL.M2.ln2_g, DL.M2.ln2_b);
   wg(row(R_dT4), row(R_U2), DL.M2.F.W2); cs(row(R_dT4), DL.M2.F.b2);
   wg(row(R_dU2), row(R_Hb2), DL.M2.F.W1); cs(row(R_dU2), DL.M2.F.b1);
-  lg(row(R_T3), row(R_dHb2), DL.M2.ln1_g, DL.M2.ln1_b);
+  lg(row(R_T3), DL.M2.ln1_g, row(R_dHb2), DL.M2.ln1_g, DL.M2.ln1_b);
   wg(row(R_dT3), row(R_O2), DL.M2.Wo); cs(row(R_dT3), DL.M2.bo);
   wg(row(R_dQ2), row(R_pma), DL.M2.Wq); cs(row(R_dQ2), DL.M2.bq);
   wg(row(R_dK2), row(R_pma), DL.M2.Wk); cs(row(R_dK2), DL.M2.bk);
   wg(row(R_dV2), row(R_pma), DL.M2.Wv); cs(row(R_dV2), DL.M2.bv);
-  lg(row(R_T2), row(R_dpma), DL.M1.ln2_g, DL.M1.ln2_b);
+  lg(row(R_T2), DL.M1.ln2_g, row(R_dpma), DL.M1.ln2_g, DL.M1.ln2_b);
   wg(row(R_dT2), row(R_U1), DL.M1.F.W2); cs(row(R_dT2), DL.M1.F.b2);
   wg(row(R_dU1), row(R_Hb1), DL.M1.F.W1); cs(row(R_dU1), DL.M1.F.b1);
-  lg(row(R_T1), row(R_dHb1), DL.M1.ln1_g, DL.M1.ln1_b);
+  lg(row(R_T1), DL.M1.ln1_g, row(R_dHb1), DL.M1.ln1_g, DL.M1.ln1_b);
   wg(row(R_dT1), row(R_O1), DL.M1.Wo); cs(row(R_dT1), DL.M1.bo);
   cs(row(R_dO1), DL.M1.bv);
   const int dh = D / cf.heads;
-  for (int h = 0; h < cf.heads; ++h) {     // ∂W_v rows of head h: Σ_(g,j) ∂O1[g,j][h] ⊗ P̄[g,(j,h)]
-    dec_rows_wgrad_kernel<<<(dh * D + 255) / 256, 256, 0, st>>>(
-        row(R_dO1) + h * dh, D, pbar + size_t(h) * D, cf.heads * D, RK, dh, D,
-        G + DL.M1.Wv + size_t(h) * dh * D, D);
-    ++n;
-  }
+  for (int h = 0; h < cf.heads; ++h)       // ∂W_v rows of head h: Σ_(g,j) ∂O1[g,j][h] ⊗ P̄[g,(j,h)]
+    if ((rr = launch_wgrad(ctx, dO1h + size_t(h) * RK * dh, dh, pbar + size_t(h) * RK * D, D, RK,
+                           G + DL.M1.Wv + size_t(h) * dh * D, st, false)) >= 0) n += rr;
   OCCU_PROF_END(ctx);
+  if (rr < 0) return rr;
   // PMA's pre-pooling FFN over the N node rows (tensor cores): Z = T W2ᵀ + b2, T = ReLU(h W1ᵀ + b1)
   int r;
+  (void)row;
   if ((r = launch_plain_masked_tc(ctx, dZ, D, csr.N, 3, cf.L, nullptr, dT, "dec_ffn_bwd_tc", st, T, 0.f)) < 0) return r;
   n += r;
   if ((r = launch_wgrad(ctx, dZ, D, T, D, csr.N, G + DL.P.W2, st, false)) < 0) return r;

@@ -407,6 +407,13 @@ int launch_colsum_rows(occu_ctx *ctx, const float *X, long R, float *out, cudaSt
   return colsum(ctx, X, R, out, st);
 }
 
+static int ln_bwd(occu_ctx *ctx, const float *x, const float *gam, const float *dy, const float *add,
+                  float *dx, long R, float *gg, float *gb, cudaStream_t st);
+int launch_ln_param_grads(occu_ctx *ctx, const float *x, const float *gam, const float *dy, long R,
+                          float *dx_scratch, float *gg, float *gb, cudaStream_t st) {
+  return ln_bwd(ctx, x, gam, dy, nullptr, dx_scratch, R, gg, gb, st);
+}
+
 // dx = add + LNᵀ(dy) for x = LN input; dγ, dβ into gg, gb.
 static int ln_bwd(occu_ctx *ctx, const float *x, const float *gam, const float *dy, const float *add,
                   float *dx, long R, float *gg, float *gb, cudaStream_t st) {

@@ -277,6 +277,10 @@ int launch_set_decoder_bwd(occu_ctx *ctx, const DevCsr &csr, const float *hL, co
                            cudaStream_t st);
 // out[c] = Σ_r X[r][c] over R rows of width d, fixed order (kernels_stack.cu)
 int launch_colsum_rows(occu_ctx *ctx, const float *X, long R, float *out, cudaStream_t st);
+// LayerNorm parameter gradients over R rows (x = LN input, gamma its gain): dγ = Σ dy ⊙ x̂,
+// dβ = Σ dy (fixed order); dx_scratch [R][d] receives the (unused) input gradient.
+int launch_ln_param_grads(occu_ctx *ctx, const float *x, const float *gam, const float *dy, long R,
+                          float *dx_scratch, float *gg, float *gb, cudaStream_t st);
 // Image slot of Graphormer layer j's transposed matrices (kinds 0-5: W_qᵀ W_kᵀ W_vᵀ W_oᵀ W1ᵀ W2ᵀ).
 int gph_tslot(const occu_config &c, int j);
 int launch_bias_add_tc(const occu_ctx *ctx, const float *A, int K, int R, int wkind, int layer,
