@@ -1409,6 +1409,117 @@ __global__ void __launch_bounds__(NT) node_bwd_kernel(
   }
 }
 
+// node_bwd with deeper memory-level parallelism (same sums, same per-node order): a warp
+// takes chunks of 8 consecutive nodes; their out_ptr / in_ptr words, h̄ rows and in-edge dα
+// sums are requested at once, then the chunk's out-edges (contiguous in out-CSR order) are
+// walked G at a time with all G MG rows in flight, and each node is flushed as its out-edge
+// segment ends (ascending out-CSR order, as node_bwd_kernel).
+template <int D, bool BF>
+__global__ void __launch_bounds__(NT, 3) node_bwd_v2_kernel(
+    const float *__restrict__ MG, const float *__restrict__ dalpha,
+    const void *__restrict__ hbar, const float *__restrict__ a_s, const float *__restrict__ a_d,
+    const int32_t *__restrict__ out_ptr, const int32_t *__restrict__ out_pos,
+    const int32_t *__restrict__ in_ptr, int N, float slope, float *__restrict__ dP,
+    float *__restrict__ dpq, float *__restrict__ da_part) {
+  constexpr int V = D / 32;
+  constexpr int NPW = 8, G = 4;
+  const int lane = threadIdx.x & 31;
+  const long nw = (long(gridDim.x) * NT) / 32;
+  double das[V], dad[V];
+  float a_sv[V], a_dv[V];
+#pragma unroll
+  for (int c = 0; c < V; ++c) {
+    das[c] = dad[c] = 0.0;
+    a_sv[c] = __ldg(a_s + lane * V + c);
+    a_dv[c] = __ldg(a_d + lane * V + c);
+  }
+  for (long t0 = (blockIdx.x * long(NT) + threadIdx.x) / 32 * NPW; t0 < N; t0 += nw * NPW) {
+    const int nn = int(min(long(NPW), N - t0));
+    const int op_l = lane <= nn ? __ldg(out_ptr + t0 + lane) : 0;
+    const int ip_l = lane <= nn ? __ldg(in_ptr + t0 + lane) : 0;
+    // h̄ row of the node being accumulated (the next one is requested at each flush) and dq
+    // of node `lane` (lane < nn)
+    RawRow<V, BF> hb;
+    hb.load(hbar, t0, D, lane);
+    float dq_l = 0.f;
+    {
+      const int ie = __shfl_down_sync(0xffffffffu, ip_l, 1);
+      if (lane < nn)
+        for (int k = ip_l; k < ie; ++k) dq_l += __ldg(dalpha + k);
+    }
+    const int e_beg = __shfl_sync(0xffffffffu, op_l, 0);
+    const int e_end = __shfl_sync(0xffffffffu, op_l, nn);
+    int node = 0;
+    int seg_end = __shfl_sync(0xffffffffu, op_l, 1);
+    float acc[V], dp = 0.f;
+#pragma unroll
+    for (int c = 0; c < V; ++c) acc[c] = 0.f;
+    auto flush = [&](int nd) {
+      float hv[V], o[V];
+      hb.get(hv);
+      if (nd + 1 < nn) hb.load(hbar, t0 + nd + 1, D, lane);
+      const float dq = __shfl_sync(0xffffffffu, dq_l, nd);
+#pragma unroll
+      for (int c = 0; c < V; ++c) {
+        const float v = acc[c] + dp * a_sv[c] + dq * a_dv[c];
+        o[c] = v * lrelu_grad_from_out(hv[c], slope);
+        das[c] = fma(double(dp), double(hv[c]), das[c]);
+        dad[c] = fma(double(dq), double(hv[c]), dad[c]);
+        acc[c] = 0.f;
+      }
+      store_row<V>(dP + (t0 + nd) * D + lane * V, o);
+      if (lane == 0) {
+        dpq[2 * (t0 + nd)] = dp;
+        dpq[2 * (t0 + nd) + 1] = dq;
+      }
+      dp = 0.f;
+    };
+    for (int base = e_beg; base < e_end; base += 32) {
+      const int cnt = min(32, e_end - base);
+      const int pos_l = lane < cnt ? __ldg(out_pos + base + lane) : 0;
+      const float da_l = lane < cnt ? __ldg(dalpha + pos_l) : 0.f;
+      for (int j = 0; j < cnt; j += G) {
+        RawRow<V, false> rr[G];
+#pragma unroll
+        for (int u = 0; u < G; ++u) rr[u].load(MG, long(__shfl_sync(0xffffffffu, pos_l, min(j + u, cnt - 1))), D, lane);
+#pragma unroll
+        for (int u = 0; u < G; ++u) {
+          const float dau = __shfl_sync(0xffffffffu, da_l, min(j + u, cnt - 1));
+          if (j + u < cnt) {
+            const int k = base + j + u;
+            while (k >= seg_end) {
+              flush(node);
+              ++node;
+              seg_end = __shfl_sync(0xffffffffu, op_l, node + 1);
+            }
+            float x[V];
+            rr[u].get(x);
+#pragma unroll
+            for (int c = 0; c < V; ++c) acc[c] += x[c];
+            dp += dau;
+          }
+        }
+      }
+    }
+    for (; node < nn; ++node) flush(node);
+  }
+  if (da_part) {   // per-block partial: warps combined in fixed warp order through smem
+    __shared__ double red[NT / 32][2 * D];
+    const int wl = threadIdx.x / 32;
+#pragma unroll
+    for (int c = 0; c < V; ++c) {
+      red[wl][lane * V + c] = das[c];
+      red[wl][D + lane * V + c] = dad[c];
+    }
+    __syncthreads();
+    for (int o = threadIdx.x; o < 2 * D; o += NT) {
+      double acc2 = 0.0;
+      for (int w2 = 0; w2 < NT / 32; ++w2) acc2 += red[w2][o];
+      da_part[long(blockIdx.x) * 2 * D + o] = float(acc2);
+    }
+  }
+}
+
 // Deterministic split-K weight gradient: partial[s][a][b] = Σ_{r in split s} X[r][a] Y[r][b]
 // (X: [R][A], Y: [R][Bn]; 128x128 output tile per CTA, 8x8 per thread).
 constexpr int WG_R = 32;
@@ -2063,7 +2174,17 @@ static int backward_layer_impl(occu_ctx *ctx, const DevCsr &csr, const BwdLayerA
   if (w.dpart.ensure(size_t(nb_blocks) * 2 * D * 4) != cudaSuccess) return -int(cudaErrorMemoryAllocation);
   float *da_part = w.dpart.as<float>();
   OCCU_PROF_BEGIN(ctx, "node_bwd", st);
-  if (bf)
+  static const int nbv = getenv("OCCU_NODE_BWD_V1") ? 0 : 1;     // A/B switch: 1 = v2 (default)
+  const int nb2 = nb_blocks;        // (the [da_s; da_d] partials are sized for nb_blocks)
+  if (nbv && bf)
+    node_bwd_v2_kernel<D, true><<<nb2, NT, 0, st>>>(
+        w.MG.as<float>(), w.dalpha.as<float>(), a.hbar, P + L.a_s[i], P + L.a_d[i], csr.out_ptr,
+        csr.out_pos, csr.in_ptr, csr.N, cf.slope, w.dP.as<float>(), w.dpq.as<float>(), da_part);
+  else if (nbv)
+    node_bwd_v2_kernel<D, false><<<nb2, NT, 0, st>>>(
+        w.MG.as<float>(), w.dalpha.as<float>(), a.hbar, P + L.a_s[i], P + L.a_d[i], csr.out_ptr,
+        csr.out_pos, csr.in_ptr, csr.N, cf.slope, w.dP.as<float>(), w.dpq.as<float>(), da_part);
+  else if (bf)
     node_bwd_kernel<D, true><<<nb_blocks, NT, 0, st>>>(
         w.MG.as<float>(), w.dalpha.as<float>(), a.hbar, P + L.a_s[i], P + L.a_d[i], csr.out_ptr,
         csr.out_pos, csr.in_ptr, csr.N, cf.slope, w.dP.as<float>(), w.dpq.as<float>(), da_part);

@@ -444,12 +444,16 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
         aux = __ldg(a.pin + __ldg(a.src + r0 + row)) + __ldg(a.qin + __ldg(a.dst + r0 + row));  // α (R1)
       // EDGEBWD: the row's first de chunk is fetched before waiting on the accumulator, and
       // every later chunk one step ahead (the epilogue is paced by these per-row loads)
+      // PLAIN: likewise the row's addend (or, without one, its FP32 mask) — the one per-row
+      // stream of the de / dh_prev GEMMs — one chunk ahead
       float4 dpre[4];
-      if (EPI == EPI_EDGEBWD) {
+      const float *pre_src = EPI == EPI_EDGEBWD ? a.de
+                           : (EPI == EPI_PLAIN ? (a.add ? a.add : (a.mask_bf ? nullptr : a.mask_h)) : nullptr);
+      if (EPI == EPI_EDGEBWD || EPI == EPI_PLAIN) {
 #pragma unroll
         for (int u = 0; u < 4; ++u)
-          dpre[u] = live ? __ldg(reinterpret_cast<const float4 *>(a.de + (r0 + row) * D + hf * (D / 2) + 4 * u))
-                         : make_float4(0.f, 0.f, 0.f, 0.f);
+          dpre[u] = (live && pre_src) ? __ldg(reinterpret_cast<const float4 *>(pre_src + (r0 + row) * D + hf * (D / 2) + 4 * u))
+                                      : make_float4(0.f, 0.f, 0.f, 0.f);
       }
       TT_WAIT_BEGIN
       tc::mbar_wait(s.eready + (i & 3), (i >> 2) & 1);
@@ -468,8 +472,19 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
       const int wrows = max(0, min(32, nrows - qd * 32));
       const uint32_t acc = lane_base + acc_col(j) + cb;
       if (EPI == EPI_PLAIN) {
+        const bool pre_add = a.add != nullptr;                 // dpre holds the addend chunk
+        const bool pre_mask = !pre_add && pre_src != nullptr;  // dpre holds the FP32 mask chunk
 #pragma unroll 1
         for (int c0 = 0; c0 < DH; c0 += 16) {
+          float4 dcur[4];
+#pragma unroll
+          for (int u = 0; u < 4; ++u) dcur[u] = dpre[u];
+          if (pre_src && c0 + 16 < DH) {
+            const float *pn = pre_src + grow * D + cb + c0 + 16;
+#pragma unroll
+            for (int u = 0; u < 4; ++u)
+              dpre[u] = live ? __ldg(reinterpret_cast<const float4 *>(pn + 4 * u)) : make_float4(0.f, 0.f, 0.f, 0.f);
+          }
           uint32_t r[16];
           tc::tmem_ld16(acc + c0, r);
           tc::tmem_ld_wait();
@@ -491,6 +506,8 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
                 const uint2 b = __ldg(reinterpret_cast<const uint2 *>(mb + u));
                 x = make_float4(__uint_as_float(b.x << 16), __uint_as_float(b.x & 0xFFFF0000u),
                                 __uint_as_float(b.y << 16), __uint_as_float(b.y & 0xFFFF0000u));
+              } else if (pre_mask) {
+                x = dcur[u >> 2];
               } else {
                 x = __ldg(reinterpret_cast<const float4 *>(mr + u));
               }
@@ -509,11 +526,10 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
               if (a.relu) o[u] = fmaxf(o[u], 0.f);
             }
           }
-          if (a.add && live) {
-            const float *ar = a.add + grow * D + cb + c0;
+          if (pre_add && live) {
 #pragma unroll
             for (int u = 0; u < 16; u += 4) {
-              const float4 x = __ldg(reinterpret_cast<const float4 *>(ar + u));
+              const float4 x = dcur[u >> 2];
               o[u] += x.x; o[u + 1] += x.y; o[u + 2] += x.z; o[u + 3] += x.w;
             }
           }
@@ -546,15 +562,21 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
             if (live && a.e) ev = __ldg(reinterpret_cast<const float4 *>(a.e + grow * D + cb + c0 + u));
             float evv[4] = {ev.x, ev.y, ev.z, ev.w};
             const float dvv[4] = {dv.x, dv.y, dv.z, dv.w};
-            if (!a.e) {
+            float sneg[4];
 #pragma unroll
-              for (int t = 0; t < 4; ++t) evv[t] = fast_rcp(1.f + ex2(__uint_as_float(r[u + t]) * cexp));
+            for (int t = 0; t < 4; ++t) {
+              // τ = e^{-y}, y = α z: σ(y) = 1/(1 + τ) (the forward's e', same bits) and
+              // σ(-y) = τ·σ(y) — one MUFU ex2 + one rcp per element; τ = inf -> σ(-y) = 1
+              const float tau = ex2(__uint_as_float(r[u + t]) * cexp);
+              const float sp = fast_rcp(1.f + tau);
+              if (!a.e) evv[t] = sp;
+              sneg[t] = tau < 3.0e38f ? tau * sp : 1.f;
             }
 #pragma unroll
             for (int t = 0; t < 4; ++t) {
               const float z = __uint_as_float(r[u + t]) * un;
               // σ'(y) = σ(y)·σ(-y), y = α z (recomputed): no 1 - e' cancellation
-              const float dy = dvv[t] * evv[t] * fast_rcp(1.f + fast_exp(aux * z));
+              const float dy = dvv[t] * evv[t] * sneg[t];
               dpart = fma(double(dy), double(z), dpart);
               o[u + t] = aux * dy;
             }
