@@ -676,7 +676,7 @@ __global__ void __launch_bounds__(NT) gate_bwd_stream_kernel(
             mg[c] = dv[c] * gv[c];
             dvv[c] = mg[c] * (hv[c] - At);
           }
-          store_row<V>(MG + (k0 + j + u) * D + lane * V, mg);
+          if (MG) store_row<V>(MG + (k0 + j + u) * D + lane * V, mg);
           store_row<V>(DV + (k0 + j + u) * D + lane * V, dvv);
           continue;
         }
@@ -695,7 +695,7 @@ __global__ void __launch_bounds__(NT) gate_bwd_stream_kernel(
           mg[c] = dv[c] * gv[c];
           dvv[c] = gv[c] * (dg[c] - dotf);
         }
-        store_row<V>(MG + (k0 + j + u) * D + lane * V, mg);
+        if (MG) store_row<V>(MG + (k0 + j + u) * D + lane * V, mg);
         store_row<V>(DV + (k0 + j + u) * D + lane * V, dvv);
       }
     }
@@ -1414,13 +1414,17 @@ __global__ void __launch_bounds__(NT) node_bwd_kernel(
 // sums are requested at once, then the chunk's out-edges (contiguous in out-CSR order) are
 // walked G at a time with all G MG rows in flight, and each node is flushed as its out-edge
 // segment ends (ascending out-CSR order, as node_bwd_kernel).
-template <int D, bool BF>
-__global__ void __launch_bounds__(NT, 3) node_bwd_v2_kernel(
+// FROMG: MG_k = dA[t_k] ⊙ g_k is formed here from the saved gates (g: BF16 rows when BF) and
+// the layer's dA instead of being written by the gate backward and read back (the same FP32
+// product, so the same bits).
+template <int D, bool BF, bool FROMG>
+__global__ void __launch_bounds__(NT, FROMG ? 2 : 3) node_bwd_v2_kernel(
     const float *__restrict__ MG, const float *__restrict__ dalpha,
     const void *__restrict__ hbar, const float *__restrict__ a_s, const float *__restrict__ a_d,
     const int32_t *__restrict__ out_ptr, const int32_t *__restrict__ out_pos,
     const int32_t *__restrict__ in_ptr, int N, float slope, float *__restrict__ dP,
-    float *__restrict__ dpq, float *__restrict__ da_part) {
+    float *__restrict__ dpq, float *__restrict__ da_part, const void *__restrict__ gsv,
+    const float *__restrict__ dA, const int32_t *__restrict__ in_dst) {
   constexpr int V = D / 32;
   constexpr int NPW = 8, G = 4;
   const int lane = threadIdx.x & 31;
@@ -1478,10 +1482,20 @@ __global__ void __launch_bounds__(NT, 3) node_bwd_v2_kernel(
       const int cnt = min(32, e_end - base);
       const int pos_l = lane < cnt ? __ldg(out_pos + base + lane) : 0;
       const float da_l = lane < cnt ? __ldg(dalpha + pos_l) : 0.f;
+      const int dst_l = (FROMG && lane < cnt) ? __ldg(in_dst + pos_l) : 0;
       for (int j = 0; j < cnt; j += G) {
         RawRow<V, false> rr[G];
+        RawRow<V, BF> gg[FROMG ? G : 1];
 #pragma unroll
-        for (int u = 0; u < G; ++u) rr[u].load(MG, long(__shfl_sync(0xffffffffu, pos_l, min(j + u, cnt - 1))), D, lane);
+        for (int u = 0; u < G; ++u) {
+          const int kk = min(j + u, cnt - 1);
+          if constexpr (FROMG) {
+            gg[u].load(gsv, long(__shfl_sync(0xffffffffu, pos_l, kk)), D, lane);
+            rr[u].load(dA, long(__shfl_sync(0xffffffffu, dst_l, kk)), D, lane);
+          } else {
+            rr[u].load(MG, long(__shfl_sync(0xffffffffu, pos_l, kk)), D, lane);
+          }
+        }
 #pragma unroll
         for (int u = 0; u < G; ++u) {
           const float dau = __shfl_sync(0xffffffffu, da_l, min(j + u, cnt - 1));
@@ -1494,6 +1508,12 @@ __global__ void __launch_bounds__(NT, 3) node_bwd_v2_kernel(
             }
             float x[V];
             rr[u].get(x);
+            if constexpr (FROMG) {
+              float gv[V];
+              gg[u].get(gv);
+#pragma unroll
+              for (int c = 0; c < V; ++c) x[c] = x[c] * gv[c];     // dm ⊙ g, as the gate backward
+            }
 #pragma unroll
             for (int c = 0; c < V; ++c) acc[c] += x[c];
             dp += dau;
@@ -2081,13 +2101,16 @@ static int backward_layer_impl(occu_ctx *ctx, const DevCsr &csr, const BwdLayerA
   const bool in_bf = bf && i > 0;           // h_in, e_in of layer 1 are the FP32 inputs
   if ((bf || cf.msg == OCCU_MSG_NEIGHBOR_SOFTMAX) && !(tc && a.g)) return -int(cudaErrorInvalidValue);
   int r;
+  // the streaming gate backward (saved gates) leaves MG = dA[t] ⊙ g to the node backward
+  const bool mg_from_g = tc && a.g && !getenv("OCCU_NODE_BWD_V1");
+  float *MGo = mg_from_g ? nullptr : w.MG.as<float>();
   if (tc && csr.E > 0) {
     // a10: softmax / message backward (streaming with the saved gates, else g recomputed on
     // tensor cores), W_mᵀ dv, z recompute + σ', W_eᵀ dz on tensor cores
     if (a.g && cf.msg == OCCU_MSG_NEIGHBOR_SOFTMAX) {
       OCCU_PROF_BEGIN(ctx, "gate_bwd", st);
       gate_bwd_stream_kernel<D, false, true><<<grid_for((long(csr.E) + 31) / 32, NT / 32, 8 * sms), NT, 0, st>>>(
-          a.g, a.dh, a.hbar, csr.in_src, csr.in_dst, csr.E, w.MG.as<float>(), w.DV.as<float>(),
+          a.g, a.dh, a.hbar, csr.in_src, csr.in_dst, csr.E, MGo, w.DV.as<float>(),
           a.h, csr.in_ptr, cf.aggr == OCCU_AGGR_MEAN, cf.slope);
       OCCU_PROF_END(ctx);
       LAUNCH_CHECK();
@@ -2096,10 +2119,10 @@ static int backward_layer_impl(occu_ctx *ctx, const DevCsr &csr, const BwdLayerA
       OCCU_PROF_BEGIN(ctx, "gate_bwd", st);
       if (bf)
         gate_bwd_stream_kernel<D, true><<<grid_for((long(csr.E) + 31) / 32, NT / 32, 8 * sms), NT, 0, st>>>(
-            a.g, a.dh, a.hbar, csr.in_src, csr.in_dst, csr.E, w.MG.as<float>(), w.DV.as<float>());
+            a.g, a.dh, a.hbar, csr.in_src, csr.in_dst, csr.E, MGo, w.DV.as<float>());
       else
         gate_bwd_stream_kernel<D, false><<<grid_for((long(csr.E) + 31) / 32, NT / 32, 8 * sms), NT, 0, st>>>(
-            a.g, a.dh, a.hbar, csr.in_src, csr.in_dst, csr.E, w.MG.as<float>(), w.DV.as<float>());
+            a.g, a.dh, a.hbar, csr.in_src, csr.in_dst, csr.E, MGo, w.DV.as<float>());
       OCCU_PROF_END(ctx);
       LAUNCH_CHECK();
       ++n;
@@ -2175,23 +2198,22 @@ static int backward_layer_impl(occu_ctx *ctx, const DevCsr &csr, const BwdLayerA
   float *da_part = w.dpart.as<float>();
   OCCU_PROF_BEGIN(ctx, "node_bwd", st);
   static const int nbv = getenv("OCCU_NODE_BWD_V1") ? 0 : 1;     // A/B switch: 1 = v2 (default)
-  const int nb2 = nb_blocks;        // (the [da_s; da_d] partials are sized for nb_blocks)
-  if (nbv && bf)
-    node_bwd_v2_kernel<D, true><<<nb2, NT, 0, st>>>(
-        w.MG.as<float>(), w.dalpha.as<float>(), a.hbar, P + L.a_s[i], P + L.a_d[i], csr.out_ptr,
-        csr.out_pos, csr.in_ptr, csr.N, cf.slope, w.dP.as<float>(), w.dpq.as<float>(), da_part);
+  const bool fromg = nbv && mg_from_g;
+#define OCCU_NB_ARGS w.MG.as<float>(), w.dalpha.as<float>(), a.hbar, P + L.a_s[i], P + L.a_d[i], csr.out_ptr, \
+    csr.out_pos, csr.in_ptr, csr.N, cf.slope, w.dP.as<float>(), w.dpq.as<float>(), da_part
+  if (fromg && bf)
+    node_bwd_v2_kernel<D, true, true><<<nb_blocks, NT, 0, st>>>(OCCU_NB_ARGS, a.g, a.dh, csr.in_dst);
+  else if (fromg)
+    node_bwd_v2_kernel<D, false, true><<<nb_blocks, NT, 0, st>>>(OCCU_NB_ARGS, a.g, a.dh, csr.in_dst);
+  else if (nbv && bf)
+    node_bwd_v2_kernel<D, true, false><<<nb_blocks, NT, 0, st>>>(OCCU_NB_ARGS, nullptr, nullptr, nullptr);
   else if (nbv)
-    node_bwd_v2_kernel<D, false><<<nb2, NT, 0, st>>>(
-        w.MG.as<float>(), w.dalpha.as<float>(), a.hbar, P + L.a_s[i], P + L.a_d[i], csr.out_ptr,
-        csr.out_pos, csr.in_ptr, csr.N, cf.slope, w.dP.as<float>(), w.dpq.as<float>(), da_part);
+    node_bwd_v2_kernel<D, false, false><<<nb_blocks, NT, 0, st>>>(OCCU_NB_ARGS, nullptr, nullptr, nullptr);
   else if (bf)
-    node_bwd_kernel<D, true><<<nb_blocks, NT, 0, st>>>(
-        w.MG.as<float>(), w.dalpha.as<float>(), a.hbar, P + L.a_s[i], P + L.a_d[i], csr.out_ptr,
-        csr.out_pos, csr.in_ptr, csr.N, cf.slope, w.dP.as<float>(), w.dpq.as<float>(), da_part);
+    node_bwd_kernel<D, true><<<nb_blocks, NT, 0, st>>>(OCCU_NB_ARGS);
   else
-    node_bwd_kernel<D, false><<<nb_blocks, NT, 0, st>>>(
-        w.MG.as<float>(), w.dalpha.as<float>(), a.hbar, P + L.a_s[i], P + L.a_d[i], csr.out_ptr,
-        csr.out_pos, csr.in_ptr, csr.N, cf.slope, w.dP.as<float>(), w.dpq.as<float>(), da_part);
+    node_bwd_kernel<D, false><<<nb_blocks, NT, 0, st>>>(OCCU_NB_ARGS);
+#undef OCCU_NB_ARGS
   OCCU_PROF_END(ctx);
   LAUNCH_CHECK();
   ++n;
