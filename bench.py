@@ -648,8 +648,8 @@ class Bench:
             N, E, B = batch.num_nodes, batch.num_edges, batch.num_graphs
             alg = algorithmic_bytes(N, E, B, d=d, rrows=readout_rows(batch.graphs))
             r = {"value": B * self.world / (ms * 1e-3), "ms_per_step": ms, "N": N, "E": E}
-            if "gather_segsum" in prof:
-                gms = prof["gather_segsum"][0] / self.args.steps
+            if "gather_segsum" in prof:      # + the hub pre-pass (part of the aggregation)
+                gms = (prof["gather_segsum"][0] + prof.get("gather_hubs", (0.0, 0))[0]) / self.args.steps
                 r["gather_segsum_GBps"] = alg["gather_segsum"] / (gms * 1e-3) / 1e9
                 r["gather_segsum_frac"] = r["gather_segsum_GBps"] / self.peaks["hbm_gbs"]
             out[name] = r

@@ -108,6 +108,10 @@ typedef struct {
   int32_t *out_pos;                       /* [E]   */
   int32_t *node_graph;                    /* [N]   */
   int32_t on_device;
+  int32_t max_in_degree;                  /* max_v (in_ptr[v+1] - in_ptr[v]); -1 = unknown.  Set
+                                             by occu_pack / occu_synthesize, kept by
+                                             occu_batch_to_device; selects the aggregation's
+                                             hub path (in-degree > 256, see occu_predict) */
   void *priv;                             /* library-private (device schedule) */
 } occu_csr_batch;
 

@@ -489,12 +489,97 @@ __device__ __forceinline__ void store_row_t(void *base, long row, int D, int lan
   }
 }
 
+// ---------------------------------------------------------------------------
+// Hub destinations (in-degree > HUB_DEG, e.g. §8(d)'s skew benchmark): one warp would walk the
+// whole segment alone, so it is split into 64-edge units first — hub_partial_kernel sums each
+// unit's share of a hub segment (ascending edge order, warp per unit, slot 0 = the unit's
+// first destination, slot 1 = its last), hub_merge_kernel adds a hub's unit partials in unit
+// order into the slot of its first unit, and gather_segsum_v2 takes that sum for the node
+// instead of walking its edges.  Fixed order throughout (deterministic, atomic-free).
+constexpr int HUB_DEG = 256, HUB_UB = 64;
+
+template <int D, bool BF>
+__global__ void __launch_bounds__(NT) hub_partial_kernel(
+    const void *__restrict__ g, const void *__restrict__ hbar, const int32_t *__restrict__ in_ptr,
+    const int32_t *__restrict__ in_src, const int32_t *__restrict__ in_dst, int E,
+    float *__restrict__ part) {
+  constexpr int V = D / 32, G = 4;
+  const int lane = threadIdx.x & 31;
+  const long nw = (long(gridDim.x) * NT) / 32;
+  const long units = (long(E) + HUB_UB - 1) / HUB_UB;
+  for (long u = (blockIdx.x * long(NT) + threadIdx.x) / 32; u < units; u += nw) {
+    const int kb = int(u * HUB_UB), ke = int(min(long(E), u * HUB_UB + HUB_UB));
+    const int t0 = __ldg(in_dst + kb), t1 = __ldg(in_dst + ke - 1);
+    for (int slot = 0; slot < 2; ++slot) {
+      const int t = slot ? t1 : t0;
+      if (slot && t1 == t0) break;
+      const int sb = __ldg(in_ptr + t), se = __ldg(in_ptr + t + 1);
+      if (se - sb <= HUB_DEG) continue;
+      const int a = max(kb, sb), b = min(ke, se);
+      float acc[V];
+#pragma unroll
+      for (int c = 0; c < V; ++c) acc[c] = 0.f;
+      for (int base = a; base < b; base += 32) {
+        const int cnt = min(32, b - base);
+        const int s_l = lane < cnt ? __ldg(in_src + base + lane) : 0;
+        for (int j = 0; j < cnt; j += G) {
+          RawRow<V, BF> gr[G], hr[G];
+#pragma unroll
+          for (int q = 0; q < G; ++q) {
+            const int kk = min(j + q, cnt - 1);
+            gr[q].load(g, long(base + kk), D, lane);
+            hr[q].load(hbar, long(__shfl_sync(0xffffffffu, s_l, kk)), D, lane);
+          }
+#pragma unroll
+          for (int q = 0; q < G; ++q)
+            if (j + q < cnt) {
+              float gv[V], hv[V];
+              gr[q].get(gv);
+              hr[q].get(hv);
+#pragma unroll
+              for (int c = 0; c < V; ++c) acc[c] = fmaf(gv[c], hv[c], acc[c]);
+            }
+        }
+      }
+      store_row<V>(part + (u * 2 + slot) * D + lane * V, acc);
+    }
+  }
+}
+
+template <int D>
+__global__ void __launch_bounds__(NT) hub_merge_kernel(const int32_t *__restrict__ in_ptr,
+                                                       const int32_t *__restrict__ in_dst, int E,
+                                                       float *__restrict__ part) {
+  constexpr int V = D / 32;
+  const int lane = threadIdx.x & 31;
+  const long nw = (long(gridDim.x) * NT) / 32;
+  const long units = (long(E) + HUB_UB - 1) / HUB_UB;
+  for (long u = (blockIdx.x * long(NT) + threadIdx.x) / 32; u < units; u += nw) {
+    const int kb = int(u * HUB_UB), ke = int(min(long(E), u * HUB_UB + HUB_UB));
+    const int t0 = __ldg(in_dst + kb), t1 = __ldg(in_dst + ke - 1);
+    for (int slot = 0; slot < 2; ++slot) {
+      const int t = slot ? t1 : t0;
+      if (slot && t1 == t0) break;
+      const int sb = __ldg(in_ptr + t), se = __ldg(in_ptr + t + 1);
+      if (se - sb <= HUB_DEG || sb / HUB_UB != u) continue;   // merged by its first unit only
+      float acc[V];
+#pragma unroll
+      for (int c = 0; c < V; ++c) acc[c] = part[(u * 2 + slot) * D + lane * V + c];
+      for (long u2 = u + 1; u2 <= (se - 1) / HUB_UB; ++u2)     // later units: t is their first dst
+#pragma unroll
+        for (int c = 0; c < V; ++c) acc[c] += part[(u2 * 2) * D + lane * V + c];
+      store_row<V>(part + (u * 2 + slot) * D + lane * V, acc);
+    }
+  }
+}
+
 template <int D, int G, bool RP, bool BF = false, bool PF = false>
-__global__ void __launch_bounds__(NT, (BF ? G <= 8 : G == 4) ? 4 : 3) gather_segsum_v2_kernel(
+__global__ void __launch_bounds__(NT, (BF ? G <= 8 : (G == 4 && !RP)) ? 4 : 3) gather_segsum_v2_kernel(
     const void *__restrict__ g, const void *__restrict__ hbar,
     const int32_t *__restrict__ in_ptr, const int32_t *__restrict__ in_src, int N, int mean,
     float slope, void *__restrict__ h_out, const int32_t *__restrict__ node_graph,
-    float *__restrict__ rpart) {
+    float *__restrict__ rpart, const float *__restrict__ hubsum = nullptr,
+    const int32_t *__restrict__ in_dst = nullptr) {
   constexpr int V = D / 32;
   constexpr int NPW = 8;
   const int lane = threadIdx.x & 31;
@@ -553,7 +638,48 @@ __global__ void __launch_bounds__(NT, (BF ? G <= 8 : G == 4) ? 4 : 3) gather_seg
     int s_l = s_first;
     int s_next = 0;
     bool next_src_issued = false;
-    for (int base = e_beg; base < e_end; base += 32) {
+    bool slow = false;
+    if (hubsum) {     // a hub in this chunk: nodes one by one, hubs from their merged unit sums
+      const int deg_l = __shfl_down_sync(0xffffffffu, ptr_l, 1) - ptr_l;
+      slow = __ballot_sync(0xffffffffu, lane < nn && deg_l > HUB_DEG) != 0u;
+    }
+    if (slow) {
+      for (int nd = 0; nd < nn; ++nd) {
+        const int kb = __shfl_sync(0xffffffffu, ptr_l, nd), ke = __shfl_sync(0xffffffffu, ptr_l, nd + 1);
+        if (ke - kb > HUB_DEG) {
+          const long u0 = kb / HUB_UB;
+          const int slot = __ldg(in_dst + u0 * HUB_UB) == int(t0 + nd) ? 0 : 1;
+#pragma unroll
+          for (int c = 0; c < V; ++c) acc[c] = hubsum[(u0 * 2 + slot) * D + lane * V + c];
+        } else {
+          for (int base = kb; base < ke; base += 32) {
+            const int cnt = min(32, ke - base);
+            const int sl = lane < cnt ? __ldg(in_src + base + lane) : 0;
+            for (int j = 0; j < cnt; j += G) {
+              RawRow<V, BF> gr[G], hr[G];
+#pragma unroll
+              for (int q = 0; q < G; ++q) {
+                const int kk = min(j + q, cnt - 1);
+                gr[q].load(g, long(base + kk), D, lane);
+                hr[q].load(hbar, long(__shfl_sync(0xffffffffu, sl, kk)), D, lane);
+              }
+#pragma unroll
+              for (int q = 0; q < G; ++q)
+                if (j + q < cnt) {
+                  float gv[V], hv[V];
+                  gr[q].get(gv);
+                  hr[q].get(hv);
+#pragma unroll
+                  for (int c = 0; c < V; ++c) acc[c] = fmaf(gv[c], hv[c], acc[c]);
+                }
+            }
+          }
+        }
+        flush(nd);
+      }
+      node = nn;
+    }
+    for (int base = e_beg; base < e_end && !slow; base += 32) {
       const int cnt = min(32, e_end - base);
       if (base > e_beg) s_l = lane < cnt ? __ldg(in_src + base + lane) : 0;
       RawRow<V, BF> gr[G], hr[G], gn[G], hn[G];
@@ -1775,6 +1901,27 @@ static int forward_layer_impl(const occu_ctx *ctx, const DevCsr &csr, const FwdL
   return n;
 }
 
+// Hub pre-pass of the aggregation (hub_partial_kernel + hub_merge_kernel) when the batch has
+// destinations of in-degree > HUB_DEG (or its maximum is unknown); *hub = the unit sums.
+template <int D, bool BF>
+static int launch_hub_sums(const occu_ctx *ctx, const DevCsr &csr, const void *g, const void *hbar,
+                           const float **hub, cudaStream_t st) {
+  *hub = nullptr;
+  if (csr.E <= 0 || (csr.max_deg >= 0 && csr.max_deg <= HUB_DEG)) return 0;
+  const long units = (long(csr.E) + HUB_UB - 1) / HUB_UB;
+  if (const_cast<occu_ctx *>(ctx)->ws.hub.ensure(size_t(units) * 2 * D * 4) != cudaSuccess)
+    return -int(cudaErrorMemoryAllocation);
+  float *part = ctx->ws.hub.as<float>();
+  const int grid = grid_for(units * 32, NT, 8 * ctx->num_sms);
+  OCCU_PROF_BEGIN(ctx, "gather_hubs", st);
+  hub_partial_kernel<D, BF><<<grid, NT, 0, st>>>(g, hbar, csr.in_ptr, csr.in_src, csr.in_dst, csr.E, part);
+  hub_merge_kernel<D><<<grid, NT, 0, st>>>(csr.in_ptr, csr.in_dst, csr.E, part);
+  OCCU_PROF_END(ctx);
+  LAUNCH_CHECK();
+  *hub = part;
+  return 2;
+}
+
 template <int D>
 static int gather_impl(const occu_ctx *ctx, const DevCsr &csr, const float *g, const float *hbar,
                        float *h_out, float *rpart, cudaStream_t st) {
@@ -1788,12 +1935,17 @@ static int gather_impl(const occu_ctx *ctx, const DevCsr &csr, const float *g, c
     return e ? atoi(e) : 8;
   }();
   const int mean = ctx->cfg.aggr == OCCU_AGGR_MEAN;
+  const float *hub = nullptr;
+  int r0 = launch_hub_sums<D, false>(ctx, csr, g, hbar, &hub, st);
+  if (r0 < 0) return r0;
   OCCU_PROF_BEGIN(ctx, "gather_segsum", st);
-#define OCCU_GATHER_ARGS g, hbar, csr.in_ptr, csr.in_src, csr.N, mean, ctx->cfg.slope, h_out, csr.node_graph, rpart
+#define OCCU_GATHER_ARGS g, hbar, csr.in_ptr, csr.in_src, csr.N, mean, ctx->cfg.slope, h_out, csr.node_graph, rpart, hub, csr.in_dst
   if (variant == 0) {
     const int grid = grid_for(long(csr.N) * 4, NT, 16 * ctx->num_sms);
-    if (rpart) gather_segsum_kernel<D, true><<<grid, NT, 0, st>>>(OCCU_GATHER_ARGS);
-    else gather_segsum_kernel<D, false><<<grid, NT, 0, st>>>(OCCU_GATHER_ARGS);
+#define OCCU_GATHER_ARGS0 g, hbar, csr.in_ptr, csr.in_src, csr.N, mean, ctx->cfg.slope, h_out, csr.node_graph, rpart
+    if (rpart) gather_segsum_kernel<D, true><<<grid, NT, 0, st>>>(OCCU_GATHER_ARGS0);
+    else gather_segsum_kernel<D, false><<<grid, NT, 0, st>>>(OCCU_GATHER_ARGS0);
+#undef OCCU_GATHER_ARGS0
   } else {
     const int grid = grid_for(long(csr.N) * 4, NT, occ * ctx->num_sms);
     if (variant == 1) {
@@ -1813,7 +1965,7 @@ static int gather_impl(const occu_ctx *ctx, const DevCsr &csr, const float *g, c
 #undef OCCU_GATHER_ARGS
   OCCU_PROF_END(ctx);
   LAUNCH_CHECK();
-  return 1;
+  return 1 + r0;
 }
 
 template <int D>
@@ -1830,8 +1982,11 @@ static int gather_bf16_impl(const occu_ctx *ctx, const DevCsr &csr, const void *
     return e ? atoi(e) : 8;
   }();
   const int grid = grid_for(long(csr.N) * 4, NT, bps * ctx->num_sms);
+  const float *hub = nullptr;
+  int r0 = launch_hub_sums<D, true>(ctx, csr, g, hbar, &hub, st);
+  if (r0 < 0) return r0;
   OCCU_PROF_BEGIN(ctx, "gather_segsum", st);
-#define OCCU_GB_ARGS g, hbar, csr.in_ptr, csr.in_src, csr.N, mean, ctx->cfg.slope, h_out, csr.node_graph, rpart
+#define OCCU_GB_ARGS g, hbar, csr.in_ptr, csr.in_src, csr.N, mean, ctx->cfg.slope, h_out, csr.node_graph, rpart, hub, csr.in_dst
   if (gsel == 4) {
     if (rpart) launch_pdl(ctx->pdl & 64, gather_segsum_v2_kernel<D, 4, true, true>, grid, NT, 0, st, OCCU_GB_ARGS);
     else launch_pdl(ctx->pdl & 64, gather_segsum_v2_kernel<D, 4, false, true>, grid, NT, 0, st, OCCU_GB_ARGS);
@@ -1845,7 +2000,7 @@ static int gather_bf16_impl(const occu_ctx *ctx, const DevCsr &csr, const void *
 #undef OCCU_GB_ARGS
   OCCU_PROF_END(ctx);
   LAUNCH_CHECK();
-  return 1;
+  return 1 + r0;
 }
 
 template <int D, bool BF>

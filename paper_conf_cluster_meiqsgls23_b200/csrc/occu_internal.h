@@ -75,11 +75,13 @@ struct Workspace {
   DevBuf gscr;             // training: Graphormer backward scratch 5 x [N][d] + stats
   DevBuf gdh[2];           // training: gradients w.r.t. the stack's node states (ping-pong)
   DevBuf dbwd;             // training: decoder backward rows / stats / partials
+  DevBuf hub;              // aggregation: per-64-edge-unit partials of hub segments
   void release_all();
 };
 
 struct DevCsr {            // device view of a packed batch
   int32_t B = 0, N = 0, E = 0;
+  int32_t max_deg = -1;    // max in-degree (-1 unknown): > HUB_DEG selects the aggregation's hub path
   const int32_t *node_off = nullptr, *edge_off = nullptr, *in_ptr = nullptr, *in_src = nullptr,
                 *in_dst = nullptr, *in_eid = nullptr, *out_ptr = nullptr, *out_pos = nullptr,
                 *node_graph = nullptr;

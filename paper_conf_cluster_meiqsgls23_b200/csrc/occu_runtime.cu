@@ -50,7 +50,7 @@ void Workspace::release_all() {
   DevBuf *bufs[] = {&node_feat, &edge_feat, &targets, &out_occ, &csr, &e0, &g, &r, &c, &yhat,
                     &dy, &dc, &dr, &dh, &dhprev, &dP, &MG, &DV, &DZ, &deA, &deB, &dalpha,
                     &dpq, &partial, &loss, &tcpart, &dpart, &rpart, &anf[0], &anf[1],
-                    &aef[0], &aef[1], &acsr[0], &acsr[1], &dT, &dZ, &dprep, &dpool, &gx, &gqkv, &go, &gscr, &gdh[0], &gdh[1], &dbwd,
+                    &aef[0], &aef[1], &acsr[0], &acsr[1], &dT, &dZ, &dprep, &dpool, &gx, &gqkv, &go, &gscr, &gdh[0], &gdh[1], &dbwd, &hub,
                     &scsr, &snf, &sef, &sdesc, &hf};
   for (DevBuf *b : bufs) b->release();
   for (auto *v : {&hbar, &p, &q, &e, &h, &gs, &gh, &gsave})
@@ -198,6 +198,7 @@ occu_status upload_csr(occu_ctx *ctx, const occu_csr_batch *b, DevBuf &dst, cuda
   out.B = b->num_graphs;
   out.N = b->num_nodes;
   out.E = b->num_edges;
+  out.max_deg = b->max_in_degree;
   if (b->on_device) {
     out.node_off = b->node_off; out.edge_off = b->edge_off; out.in_ptr = b->in_ptr;
     out.in_src = b->in_src; out.in_dst = b->in_dst; out.in_eid = b->in_eid;

@@ -294,6 +294,9 @@ extern "C" occu_status occu_pack(const occu_graph_view *graphs, int32_t num_grap
       occu_host_batch_release(b);
       return OCCU_EINVAL;
     }
+  int32_t md = 0;
+  for (int64_t v = 0; v < N; ++v) md = std::max(md, b->in_ptr[v + 1] - b->in_ptr[v]);
+  b->max_in_degree = md;
   *out = b;
   return OCCU_OK;
 }

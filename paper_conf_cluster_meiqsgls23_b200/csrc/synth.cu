@@ -23,6 +23,7 @@
 
 struct occu_template {
   int32_t n, m;
+  int32_t max_in_degree;
   int device;
   void *dmem;               // one device allocation holding everything below
   const int32_t *in_ptr, *in_src, *in_dst, *in_eid, *out_ptr, *out_pos;
@@ -212,6 +213,7 @@ extern "C" occu_status occu_template_create(occu_ctx *ctx, const occu_graph_view
   memcpy(ip + 2 * (n + 1) + m, h->in_dst, m * 4);
   memcpy(ip + 2 * (n + 1) + 2 * m, h->in_eid, m * 4);
   memcpy(ip + 2 * (n + 1) + 3 * m, h->out_pos, m * 4);
+  const int32_t tmaxdeg = h->max_in_degree;
   occu_batch_free(h);
   memcpy(ip + 2 * (n + 1) + 4 * m, codes.data(), codes.size() * 4);
   if (nd) memcpy(hbuf.data() + off_d, packed.data(), nd * 8);
@@ -227,6 +229,7 @@ extern "C" occu_status occu_template_create(occu_ctx *ctx, const occu_graph_view
   }
   occu_template *t = new occu_template;
   t->n = int32_t(n);
+  t->max_in_degree = tmaxdeg;
   t->m = int32_t(m);
   t->device = ctx->device;
   t->dmem = d;
@@ -263,6 +266,7 @@ extern "C" occu_status occu_synthesize(occu_ctx *ctx, const occu_template *const
   std::vector<SynthGraph> gs(num_graphs);
   int64_t N = 0, E = 0;
   int slices = 1;
+  int32_t maxdeg = 0;
   for (int b = 0; b < num_graphs; ++b) {
     const occu_template *t = templates[b];
     if (!t) return fail(ctx, OCCU_EINVAL, "occu_synthesize: NULL template");
@@ -281,6 +285,7 @@ extern "C" occu_status occu_synthesize(occu_ctx *ctx, const occu_template *const
     N += t->n;
     E += t->m;
     slices = std::max(slices, std::max((t->n + SN - 1) / SN, (t->m + SE - 1) / SE));
+    maxdeg = std::max(maxdeg, t->max_in_degree);
     if (N >= INT32_MAX || E >= INT32_MAX) return fail(ctx, OCCU_EINVAL, "occu_synthesize: N or E >= 2^31");
   }
   Workspace &w = ctx->ws;
@@ -310,6 +315,7 @@ extern "C" occu_status occu_synthesize(occu_ctx *ctx, const occu_template *const
   c->out_pos = q; q += E;
   c->node_graph = q;
   c->on_device = 1;
+  c->max_in_degree = maxdeg;
   c->priv = nullptr;          // arrays are ctx-owned (valid until the next occu_synthesize)
   OCCU_PROF_BEGIN(ctx, "synthesize", ctx->stream);
   synth_kernel<<<dim3(num_graphs, slices), ST, 0, ctx->stream>>>(

@@ -62,7 +62,7 @@ class CsrBatch(C.Structure):
                 ("in_dst", C.POINTER(C.c_int32)), ("in_eid", C.POINTER(C.c_int32)),
                 ("out_ptr", C.POINTER(C.c_int32)), ("out_pos", C.POINTER(C.c_int32)),
                 ("node_graph", C.POINTER(C.c_int32)), ("on_device", C.c_int32),
-                ("priv", C.c_void_p)]
+                ("max_in_degree", C.c_int32), ("priv", C.c_void_p)]
 
 
 class BatchStruct(C.Structure):

@@ -504,3 +504,38 @@ def test_save_and_load_state_resume_bitwise(tmp_path):
     m4.init_weights(1)
     with pytest.raises(occu.OccuError):
         m4.load_state(str(tmp_path / "s.bin"))
+
+
+@pytest.mark.parametrize("prec", [occu.FP32, occu.BF16], ids=["fp32", "bf16"])
+def test_hub_path_matches_oracle_and_is_deterministic(prec):
+    """§8(d)'s skew workload (1 % of nodes turned into in-degree-1,024 hubs): destinations of
+    in-degree > 256 take the aggregation's hub path (64-edge unit partials merged in unit
+    order); ŷ and r against the oracle (FP32 1e-4, BF16 per R25), both with and without kept
+    states (readout folded into the last aggregation), and reruns bitwise equal."""
+    from occu_gen import micro
+    c = occu.config(L=3, F_n=80, F_e=4, d=128, prec=prec)
+    b = micro.skew(configs.cfg2(6), seed=1006)
+    flat = weights.unit_scale(wcfg(c), weights.init_flat(wcfg(c), 42))
+    m = occu.Model(c)
+    m.set_params(flat)
+    csr = occu.pack(b.graphs)
+    assert csr.struct.max_in_degree > 256
+    y = m.predict(csr, b.node_feat, b.edge_feat)
+    assert np.array_equal(y, m.predict(csr, b.node_feat, b.edge_feat))
+    m.keep_intermediates(True)
+    yk = m.predict(csr, b.node_feat, b.edge_feat)
+    params = oracle.unflatten(ocfg(c), flat.astype(np.float64))
+    pk = oracle.pack(b.graphs)
+    ref = (oracle.forward(params, ocfg(c), pk, b.node_feat, b.edge_feat) if prec == occu.FP32
+           else oracle.forward_bf16(params, ocfg(c), pk, b.node_feat, b.edge_feat))
+    yr = ref["yhat"]
+    for yy in (y, yk):
+        if prec == occu.FP32:
+            assert np.all(np.abs(yy - yr) <= TOL * np.maximum(np.abs(yr), 1e-2))
+        else:
+            assert np.all(np.abs(yy - yr) <= 1e-2 * np.maximum(np.abs(yr), 0.1))
+    if prec == occu.FP32:
+        for i in range(c.L):
+            got = m.get_tensor(occu.T_H, i, (pk["num_nodes"], c.d))
+            assert rel(got, ref["layers"][i]["h"]) <= TOL
+            rows_ok(got, ref["layers"][i]["h"], TOL, ("h", i))
