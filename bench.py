@@ -766,15 +766,14 @@ class Bench:
         del m, csr
 
     def sec_cfg1(self):
+        """CFG1: one LeNet-5 training graph, L=2, d=64, FP32 forward; latency per graph for the
+        single-CTA kernel (the default for tiny batches) and the regular 9-kernel path, each
+        eager and replayed from a CUDA graph."""
         from occu_gen import configs
         occu, torch = self.occu, self.torch
         b1 = configs.cfg1()
-        m1 = self.model(L=2, d=64)
-        m1.init_weights(42)
-        csr1 = m1.to_device(occu.pack(b1.graphs))
         nf1 = torch.from_numpy(b1.node_feat).to(self.dev)
         ef1 = torch.from_numpy(b1.edge_feat).to(self.dev)
-        out1 = torch.empty(1, dtype=torch.float32, device=self.dev)
         reps = 1000
 
         def lat(fn):
@@ -783,50 +782,40 @@ class Bench:
             torch.cuda.synchronize()
             e0 = torch.cuda.Event(enable_timing=True)
             e1 = torch.cuda.Event(enable_timing=True)
-            e0.record(self.stream)
+            e0.record()
             for _ in range(reps):
                 fn()
-            e1.record(self.stream)
+            e1.record()
             torch.cuda.synchronize()
             return self.max_over_ranks(e0.elapsed_time(e1) * 1e3 / reps)
 
-        f1 = lambda: m1.predict(csr1, nf1, ef1, out1)
-        us = lat(f1)
-        det = {"us_per_graph": us, "launches_per_forward": m1.last_launch_count(),
-               "N": b1.num_nodes, "E": b1.num_edges}
-        try:      # the same forward captured once into a CUDA graph and replayed
+        det = {"N": b1.num_nodes, "E": b1.num_edges}
+        for small in (True, False):
+            tag = "single_cta" if small else "nine_kernel"
             side = torch.cuda.Stream(self.dev)
-            m1g = occu.Model(occu.config(L=2, F_n=80, F_e=4, d=64), device=self.local,
-                             stream=side.cuda_stream)
-            m1g.init_weights(42)
-            og = torch.empty(1, dtype=torch.float32, device=self.dev)
+            m1 = occu.Model(occu.config(L=2, F_n=80, F_e=4, d=64), device=self.local,
+                            stream=side.cuda_stream)
+            m1.init_weights(42)
+            m1.set_small_batch_kernel(small)
+            csr1 = m1.to_device(occu.pack(b1.graphs))
+            o1 = torch.empty(1, dtype=torch.float32, device=self.dev)
             with torch.cuda.stream(side):
+                det[tag + "_eager_us"] = lat(lambda: m1.predict(csr1, nf1, ef1, o1))
                 for _ in range(3):
-                    m1g.predict(csr1, nf1, ef1, og)
+                    m1.predict(csr1, nf1, ef1, o1)
+            det[tag + "_launches"] = m1.last_launch_count()
             torch.cuda.synchronize()
-            cg = torch.cuda.CUDAGraph()
-            with torch.cuda.graph(cg, stream=side):
-                m1g.predict(csr1, nf1, ef1, og)
-            torch.cuda.synchronize()
-            cg.replay()
-            torch.cuda.synchronize()
-            assert torch.equal(og, out1), "graph replay differs from the eager forward"
-            det["cuda_graph_us_per_graph"] = lat(cg.replay)
-            del cg, m1g
-        except Exception as ex:                       # noqa: BLE001 — reported, not hidden
-            det["cuda_graph"] = {"unavailable": str(ex)[:200]}
-        m1.set_small_batch_kernel(True)
-        det["single_cta_us_per_graph"] = lat(f1)
-        m1.set_small_batch_kernel(False)
-        best = min(v for k, v in det.items() if k.endswith("us_per_graph"))
+            try:
+                cg = torch.cuda.CUDAGraph()
+                with torch.cuda.graph(cg, stream=side):
+                    m1.predict(csr1, nf1, ef1, o1)
+                det[tag + "_graph_us"] = lat(cg.replay)
+                del cg
+            except Exception as ex:                   # noqa: BLE001 — reported, not hidden
+                det[tag + "_graph"] = {"unavailable": str(ex)[:200]}
+            del m1
+        best = min(v for k, v in det.items() if k.endswith("_us"))
         self.put("cfg1_latency_us", best, "f32", det, unit="us/graph")
-
-    def _templates(self, m, fams=None):
-        from occu_gen import configs
-        from occu_gen import templates as tmpl_mod
-        if not hasattr(self, "_host_tmpl"):
-            self._host_tmpl = {f: tmpl_mod.build_template(f) for f in configs.MIXTURE}
-        return [m.template(self._host_tmpl[f]) for f in (fams or configs.MIXTURE)]
 
     def sec_cfg4(self):
         """CFG4: the FULL 50,000-graph data-parallel training epoch on the 20-family mixture.

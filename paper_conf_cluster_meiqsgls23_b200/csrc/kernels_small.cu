@@ -33,11 +33,22 @@ struct SmallArgs {
 
 __device__ __forceinline__ float lrelu_s(float x, float s) { return x > 0.f ? x : s * x; }
 
-// Every global -> shared copy is a 4-byte cp.async (no register round trip, all in flight at
-// once); weights land with row stride K + 1 (the thread-per-output GEMM reads W[n][k] for 32
-// consecutive n: conflict-free).
+#ifdef OCCU_SMALL_TIMING
+__device__ unsigned long long g_small_ts[64];
+#define STAMP(i) do { if (threadIdx.x == 0 && ts_n < 64) g_small_ts[ts_n++] = (unsigned long long)(i) << 56 | (clock64() & 0xFFFFFFFFFFFFFFull); } while (0)
+#else
+#define STAMP(i) do { } while (0)
+#endif
+
+// Global -> shared copies are cp.async (no register round trip, all in flight at once); weight
+// matrices [Nout][K] land row-major with row stride K + 4 through 16-byte copies (K % 4 == 0,
+// config validation), so the GEMM reads 4 consecutive k of one output with one 16-byte load.
 __device__ __forceinline__ void cpa4(void *dst, const void *src) {
   asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(static_cast<uint32_t>(__cvta_generic_to_shared(dst))),
+               "l"(src) : "memory");
+}
+__device__ __forceinline__ void cpa16(void *dst, const void *src) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(static_cast<uint32_t>(__cvta_generic_to_shared(dst))),
                "l"(src) : "memory");
 }
 __device__ __forceinline__ void cpa_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
@@ -45,28 +56,43 @@ template <int N>
 __device__ __forceinline__ void cpa_wait() { asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory"); }
 
 __device__ __forceinline__ void stage_w(const float *__restrict__ W, int Nout, int K, float *Ws) {
-  for (int i = threadIdx.x; i < Nout * K; i += ST) cpa4(Ws + (i / K) * (K + 1) + i % K, W + i);
+  const int K4 = K / 4;
+  if ((reinterpret_cast<uintptr_t>(W) & 15) == 0) {
+    for (int i = threadIdx.x; i < Nout * K4; i += ST) {
+      const int n = i / K4, k4 = i - n * K4;
+      cpa16(Ws + n * (K + 4) + 4 * k4, W + n * K + 4 * k4);
+    }
+  } else {
+    for (int i = threadIdx.x; i < Nout * K; i += ST) cpa4(Ws + (i / K) * (K + 4) + i % K, W + i);
+  }
   cpa_commit();
 }
 
-// Y[r][n] = Σ_k X[r][k] Ws[n][k] over rows r < R, outputs n < Nout; thread per (r, n), four
-// independent partial sums, fixed order.
+// Y[r][n] = Σ_k X[r][k] Ws[n][k] over rows r < R, outputs n < Nout (K % 4 == 0); thread per
+// (4-row block, output): one 16-byte weight load per 4 k serves four rows and the four input
+// loads are warp broadcasts (a warp = 32 outputs of one row block), so shared-memory traffic
+// is ~R·Nout·K bytes instead of 4x that; k ascending (fixed order).
 __device__ __forceinline__ void small_gemm(const float *X, int ldx, int R, int K, const float *Ws,
                                            int Nout, float *Y, int ldy) {
-  for (int i = threadIdx.x; i < R * Nout; i += ST) {
-    const int r = i / Nout, n = i % Nout;
-    const float *x = X + r * ldx;
-    const float *w = Ws + n * (K + 1);
-    float a0 = 0.f, a1 = 0.f, a2 = 0.f, a3 = 0.f;
-    int k = 0;
-    for (; k + 3 < K; k += 4) {
-      a0 = fmaf(x[k], w[k], a0);
-      a1 = fmaf(x[k + 1], w[k + 1], a1);
-      a2 = fmaf(x[k + 2], w[k + 2], a2);
-      a3 = fmaf(x[k + 3], w[k + 3], a3);
+  const int ldw = K + 4, rblocks = (R + 3) / 4;
+  for (int i = threadIdx.x; i < rblocks * Nout; i += ST) {
+    const int rb = i / Nout, n = i - rb * Nout, r0 = rb * 4;
+    const float *w = Ws + n * ldw;
+    const float *x[4];
+#pragma unroll
+    for (int j = 0; j < 4; ++j) x[j] = X + min(r0 + j, R - 1) * ldx;
+    float a[4] = {0.f, 0.f, 0.f, 0.f};
+    for (int k = 0; k < K; k += 4) {
+      const float4 v = *reinterpret_cast<const float4 *>(w + k);
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        const float4 u = *reinterpret_cast<const float4 *>(x[j] + k);
+        a[j] = fmaf(u.w, v.w, fmaf(u.z, v.z, fmaf(u.y, v.y, fmaf(u.x, v.x, a[j]))));
+      }
     }
-    for (; k < K; ++k) a0 = fmaf(x[k], w[k], a0);
-    Y[r * ldy + n] = (a0 + a1) + (a2 + a3);
+#pragma unroll
+    for (int j = 0; j < 4; ++j)
+      if (r0 + j < R) Y[(r0 + j) * ldy + n] = a[j];
   }
 }
 
@@ -80,11 +106,19 @@ __global__ void __launch_bounds__(ST, 1) small_forward_kernel(const SmallArgs a)
   float *Ev = E0 + E * a.F_e;                  // [E][d]  z / logits / gates
   float *Ea = Ev + E * d;                      // [E][d]  e' (ping)
   float *Eb = Ea + E * d;                      // [E][d]  e' (pong)
-  float *Wa = Eb + E * d;                      // [d][SK + 1] weight slot A (W_u, W_m)
-  float *Wb = Wa + d * (SK + 1);               // [d][SK + 1] weight slot B (W_e)
-  int32_t *cs = reinterpret_cast<int32_t *>(Wb + d * (SK + 1));
+  float *Wa = Eb + E * d;                      // [d][SK + 4] weight slot A (W_u, W_m)
+  float *Wb = Wa + d * (SK + 4);               // [d][SK + 4] weight slot B (W_e)
+  float *W1s = Wb + d * (SK + 4);              // [d_h][d] head W_1, then b_1 [d_h], w_2 [d_h]
+  float *Rs = W1s + a.d_h * d + 2 * a.d_h;     // [B][d] readout
+  float *Cs = Rs + a.B * d;                    // [B][d_h] head hidden
+  float *Av = Cs + a.B * a.d_h;                // [L][2][d] attention vectors a_s, a_d
+  int32_t *cs = reinterpret_cast<int32_t *>(Av + a.L * 2 * d);
   int32_t *iptr = cs, *isrc = cs + (N + 1), *idst = isrc + E, *ieid = idst + E;
   const int t = threadIdx.x, warp = t >> 5, lane = t & 31;
+#ifdef OCCU_SMALL_TIMING
+  int ts_n = 0;
+#endif
+  STAMP(0);
   pdl_trigger();
   pdl_wait();
   // a1: CSR, node features, first layer's weights; then the in-CSR-ordered edge features
@@ -95,11 +129,21 @@ __global__ void __launch_bounds__(ST, 1) small_forward_kernel(const SmallArgs a)
     cpa4(ieid + i, a.in_eid + i);
   }
   for (int i = t; i < N * a.F_n; i += ST) cpa4(H + (i / a.F_n) * SK + i % a.F_n, a.nf + i);
+  // the attention vectors of every layer and the head's parameters ride in the first group
+  for (int i = t; i < a.L * 2 * d; i += ST) {
+    const int l = i / (2 * d), j = i % (2 * d);
+    cpa4(Av + i, a.P + (j < d ? a.a_s[l] + j : a.a_d[l] + j - d));
+  }
+  for (int i = t; i < a.d_h * d; i += ST) cpa4(W1s + i, a.P + a.W_1 + i);
+  for (int i = t; i < a.d_h; i += ST) {
+    cpa4(W1s + a.d_h * d + i, a.P + a.b_1 + i);
+    cpa4(W1s + a.d_h * d + a.d_h + i, a.P + a.w_2 + i);
+  }
   cpa_commit();
   stage_w(a.P + a.W_u[0], d, a.F_n, Wa);
   stage_w(a.P + a.W_e[0], d, a.F_e, Wb);
   cpa_wait<2>();                               // CSR + node features
-  __syncthreads();
+  __syncthreads(); STAMP(1);
   for (int i = t; i < E * a.F_e; i += ST) {
     const int k = i / a.F_e, c = i % a.F_e;
     cpa4(E0 + i, a.ef + size_t(ieid[k]) * a.F_e + c);
@@ -115,17 +159,17 @@ __global__ void __launch_bounds__(ST, 1) small_forward_kernel(const SmallArgs a)
     // layer 0: W_u0 is the second of four groups (CSR + H, W_u0, W_e0, E0); later layers:
     // W_u(l) is the most recent group (issued after W_e(l)), so everything must land
     if (l == 0) cpa_wait<2>(); else cpa_wait<0>();
-    __syncthreads();
+    __syncthreads(); STAMP(2);
     small_gemm(H, SK, N, K, Wa, d, Hb, d);
-    __syncthreads();
+    __syncthreads(); STAMP(3);
     stage_w(P + a.W_m[l], d, d, Wa);           // slot A: W_m (W_u consumed)
     for (int i = t; i < N * d; i += ST) Hb[i] = lrelu_s(Hb[i], a.slope);
-    __syncthreads();
+    __syncthreads(); STAMP(4);
     for (int u = warp; u < N; u += ST / 32) {
       float ps = 0.f, qs = 0.f;
       for (int c = lane; c < d; c += 32) {
-        ps = fmaf(Hb[u * d + c], __ldg(P + a.a_s[l] + c), ps);
-        qs = fmaf(Hb[u * d + c], __ldg(P + a.a_d[l] + c), qs);
+        ps = fmaf(Hb[u * d + c], Av[l * 2 * d + c], ps);
+        qs = fmaf(Hb[u * d + c], Av[l * 2 * d + d + c], qs);
       }
 #pragma unroll
       for (int o = 16; o > 0; o >>= 1) {
@@ -139,20 +183,20 @@ __global__ void __launch_bounds__(ST, 1) small_forward_kernel(const SmallArgs a)
     }
     // a3: z = e_in W_eᵀ, e' = σ(α z), α = p[src] + q[dst]     (groups: W_e[, E0], W_m)
     cpa_wait<1>();
-    __syncthreads();
+    __syncthreads(); STAMP(5);
     small_gemm(Ein, lde, E, Ke, Wb, d, Ev, d);
-    __syncthreads();
+    __syncthreads(); STAMP(6);
     if (l + 1 < a.L) stage_w(P + a.W_e[l + 1], d, d, Wb);      // slot B: next W_e
     for (int i = t; i < E * d; i += ST) {
       const int k = i / d;
       const float al = pq[isrc[k]] + pq[SNMAX + idst[k]];
-      Eout[i] = 1.f / (1.f + expf(-al * Ev[i]));
+      Eout[i] = __frcp_rn(1.f + exp2f(-al * Ev[i] * 1.4426950408889634f));
     }
     // a4: logits W_m e', softmax over the d channels (warp per edge)
     if (l + 1 < a.L) cpa_wait<1>(); else cpa_wait<0>();
-    __syncthreads();
+    __syncthreads(); STAMP(7);
     small_gemm(Eout, d, E, d, Wa, d, Ev, d);
-    __syncthreads();
+    __syncthreads(); STAMP(8);
     if (l + 1 < a.L) stage_w(P + a.W_u[l + 1], d, d, Wa);      // slot A: next W_u
     for (int k = warp; k < E; k += ST / 32) {
       float m = -INFINITY;
@@ -161,7 +205,7 @@ __global__ void __launch_bounds__(ST, 1) small_forward_kernel(const SmallArgs a)
       for (int o = 16; o > 0; o >>= 1) m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, o));
       float s = 0.f;
       for (int c = lane; c < d; c += 32) {
-        const float x = expf(Ev[k * d + c] - m);
+        const float x = exp2f((Ev[k * d + c] - m) * 1.4426950408889634f);
         Ev[k * d + c] = x;
         s += x;
       }
@@ -170,7 +214,7 @@ __global__ void __launch_bounds__(ST, 1) small_forward_kernel(const SmallArgs a)
       const float inv = 1.f / s;
       for (int c = lane; c < d; c += 32) Ev[k * d + c] *= inv;
     }
-    __syncthreads();
+    __syncthreads(); STAMP(9);
     // a5/a6: h[t] = LReLU(Σ_{k∈seg(t)} g_k ⊙ h̄[s_k]) (÷ deg for MEAN), ascending k
     for (int i = t; i < N * d; i += ST) {
       const int v = i / d, c = i % d;
@@ -180,38 +224,40 @@ __global__ void __launch_bounds__(ST, 1) small_forward_kernel(const SmallArgs a)
       if (a.mean) acc /= float(k1 > k0 ? k1 - k0 : 1);
       H[v * SK + c] = lrelu_s(acc, a.slope);
     }
-    __syncthreads();
+    __syncthreads(); STAMP(10);
     Ein = Eout;                                // e' feeds the next layer (ping-pong)
     lde = d;
     Eout = Eout == Ea ? Eb : Ea;
     K = d;
     Ke = d;
   }
-  // a7: per-graph mean readout; a8: head (warp per graph for the final dot)
+  // a7: per-graph mean readout (shared memory); a8: head, warp per hidden unit (lanes over the
+  // d channels, fixed butterfly), then warp per graph for the final dot
   for (int i = t; i < a.B * d; i += ST) {
     const int b = i / d, c = i % d;
     const int u0 = __ldg(a.node_off + b), u1 = __ldg(a.node_off + b + 1);
     float s = 0.f;
     for (int u = u0; u < u1; ++u) s += H[u * SK + c];
-    a.r[i] = s / float(u1 - u0);
+    Rs[i] = s / float(u1 - u0);
+    a.r[i] = Rs[i];
   }
-  __syncthreads();
-  for (int i = t; i < a.B * a.d_h; i += ST) {
-    const int b = i / a.d_h, n = i % a.d_h;
-    float s0 = __ldg(a.P + a.b_1 + n), s1 = 0.f, s2 = 0.f, s3 = 0.f;
-    const float *w = a.P + a.W_1 + size_t(n) * d, *rr = a.r + b * d;
-    for (int c = 0; c < d; c += 4) {
-      s0 = fmaf(__ldg(w + c), rr[c], s0);
-      s1 = fmaf(__ldg(w + c + 1), rr[c + 1], s1);
-      s2 = fmaf(__ldg(w + c + 2), rr[c + 2], s2);
-      s3 = fmaf(__ldg(w + c + 3), rr[c + 3], s3);
+  __syncthreads(); STAMP(11);
+  for (int o = warp; o < a.B * a.d_h; o += ST / 32) {
+    const int b = o / a.d_h, n = o % a.d_h;
+    float s = 0.f;
+    for (int c = lane; c < d; c += 32) s = fmaf(W1s[n * d + c], Rs[b * d + c], s);
+#pragma unroll
+    for (int q = 16; q > 0; q >>= 1) s += __shfl_xor_sync(0xffffffffu, s, q);
+    if (lane == 0) {
+      s += W1s[a.d_h * d + n];
+      Cs[o] = s;
+      a.c[o] = s;
     }
-    a.c[i] = (s0 + s1) + (s2 + s3);
   }
-  __syncthreads();
+  __syncthreads(); STAMP(12);
   for (int b = warp; b < a.B; b += ST / 32) {
     float s = 0.f;
-    for (int n = lane; n < a.d_h; n += 32) s = fmaf(__ldg(a.P + a.w_2 + n), lrelu_s(a.c[b * a.d_h + n], a.slope), s);
+    for (int n = lane; n < a.d_h; n += 32) s = fmaf(W1s[a.d_h * d + a.d_h + n], lrelu_s(Cs[b * a.d_h + n], a.slope), s);
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
     if (lane == 0) a.yhat[b] = s + __ldg(a.P + a.b_2);
@@ -223,7 +269,7 @@ __global__ void __launch_bounds__(ST, 1) small_forward_kernel(const SmallArgs a)
 static size_t small_smem(const occu_config &c, const DevCsr &csr) {
   const int sk = std::max(c.F_n, std::max(c.F_e, c.d));
   return size_t(csr.N * sk + csr.N * c.d + 2 * SNMAX + csr.E * c.F_e + 3 * csr.E * c.d +
-                2 * c.d * (sk + 1) + (csr.N + 1) + 3 * csr.E) * 4;
+                2 * c.d * (sk + 4) + c.d_h * c.d + 2 * c.d_h + csr.B * (c.d + c.d_h) + c.L * 2 * c.d + (csr.N + 1) + 3 * csr.E) * 4;
 }
 
 bool small_forward_ok(const occu_ctx *ctx, const DevCsr &csr) {
@@ -261,3 +307,10 @@ int launch_small_forward(const occu_ctx *ctx, const DevCsr &csr, const float *nf
 }
 
 }  // namespace occu
+
+#ifdef OCCU_SMALL_TIMING
+extern "C" int occu_debug_small_ts(unsigned long long *host) {
+  cudaDeviceSynchronize();
+  return int(cudaMemcpyFromSymbol(host, occu::g_small_ts, sizeof(unsigned long long) * 64));
+}
+#endif

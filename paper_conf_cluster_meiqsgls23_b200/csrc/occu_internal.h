@@ -134,7 +134,7 @@ struct occu_ctx {
   bool have_forward = false;
   bool h_last_stored = true;   // false: the last forward kept only readout partials of h_L
   bool small_fwd = false;      // the last forward ran the single-CTA small-batch kernel
-  bool small_enabled = false;  // occu_set_small_batch_kernel: single-CTA forward for tiny batches
+  bool small_enabled = true;   // occu_set_small_batch_kernel: single-CTA forward for tiny batches (default on)
   int64_t launches = 0;
   mutable occu::Profiler prof;
   // occu_predict_async: H2D on a copy stream into staging slot a_slot, compute on `stream`
