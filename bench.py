@@ -513,13 +513,35 @@ class Bench:
         for _ in range(a.steps):
             e2e_step()
         torch.cuda.synchronize()
+        e2e_sync_ms = self.max_over_ranks((time.perf_counter() - t0) * 1e3 / a.steps)
+        # pipelined through occu_train_step_async: while step k runs, the host packs batch k+1
+        # and its copies (copy stream, double-buffered staging) overlap step k; every step still
+        # packs its CSR, copies CSR + features + targets H2D and reads its loss back D2H
+        pin_loss = [torch.zeros(1).pin_memory() for _ in range(2)]
+
+        def e2e_async(k):
+            hc = occu.pack_arrays(g_nn, g_ne, g_src, g_dst)
+            m.train_step_async(hc, pin_nf, pin_ef, pin_y, LR, global_num_graphs=gB,
+                               out_loss=pin_loss[k & 1])
+
+        for k in range(a.warmup):
+            e2e_async(k)
+        m.wait()
+        self.bar()
+        t0 = time.perf_counter()
+        for k in range(a.steps):
+            e2e_async(k)
+        m.wait()
         e2e_ms = self.max_over_ranks((time.perf_counter() - t0) * 1e3 / a.steps)
         csr_bytes = 4 * (2 * (B + 1) + 2 * (N + 1) + 4 * E + N)
         e2e = {"value": gB / (e2e_ms * 1e-3), "unit": "graphs/s", "ms_per_step": e2e_ms,
                "h2d_bytes_per_step": int(b3.node_feat.nbytes + b3.edge_feat.nbytes
                                          + b3.targets.nbytes + csr_bytes),
                "d2h_bytes_per_step": 4,
-               "includes": "occu_pack + occu_train_step(host pinned buffers) + loss D2H, blocking"}
+               "synchronous_ms_per_step": e2e_sync_ms,
+               "includes": "per step: occu_pack (host C++) + occu_train_step_async (pinned host "
+                           "features / targets, H2D on the copy stream) + loss D2H, pipelined "
+                           "across steps; timed to occu_wait"}
         self.details["cfg3_f32"] = {"kernels": kernels, "roofline": roof, "loss_first": loss0,
                                     "loss_after": loss_after, "e2e": e2e, "clocks": clocks,
                                     "step_algorithmic_bytes": tot_alg}

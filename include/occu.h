@@ -167,7 +167,7 @@ occu_status occu_predict(occu_ctx *ctx, const occu_csr_batch *csr_batch,
  * batch (use occu_predict, which is already stream-ordered for those). */
 occu_status occu_predict_async(occu_ctx *ctx, const occu_csr_batch *csr_batch,
                                const float *node_feat, const float *edge_feat, float *out_occ);
-/* Blocks until every occu_predict_async issued on ctx has completed. */
+/* Blocks until every occu_predict_async / occu_train_step_async issued on ctx has completed. */
 occu_status occu_wait(occu_ctx *ctx);
 
 /* ---- training (P209-P213, P273) ------------------------------------------- */
@@ -177,6 +177,15 @@ occu_status occu_wait(occu_ctx *ctx);
  * the features' memory space; out_loss (nullable, host) = global mean loss. */
 occu_status occu_train_step(occu_ctx *ctx, const occu_batch *batch, const float *targets,
                             float lr, float *out_loss);
+/* Pipelined occu_train_step: a HOST batch (occu_pack) with pinned host features / targets;
+ * the copies run on a copy stream into one of two staging slots and the step is enqueued on
+ * the ctx stream behind them, so the host can pack the next batch and its copies overlap this
+ * step.  Blocks only until the previous call's copies have landed: keep batch, features and
+ * targets alive and unmodified until the next occu_train_step_async (or occu_wait) returns.
+ * out_loss (nullable, pinned host float) receives the global mean loss — read it after
+ * occu_wait.  Same arithmetic as occu_train_step (bitwise-identical parameters). */
+occu_status occu_train_step_async(occu_ctx *ctx, const occu_batch *batch, const float *targets,
+                                  float lr, float *out_loss);
 /* Forward + backward only (no allreduce, no Adam): grads left in the ctx. */
 occu_status occu_compute_grads(occu_ctx *ctx, const occu_batch *batch, const float *targets,
                                float *out_loss);

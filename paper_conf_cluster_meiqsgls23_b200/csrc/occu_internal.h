@@ -63,7 +63,8 @@ struct Workspace {
   DevBuf dy, dc, dr, dh, dhprev, dP, MG, DV, DZ, deA, deB, dalpha, dpq, partial, loss;
   DevBuf tcpart;           // tensor-core aggregation: boundary-segment partials
   DevBuf dpart;            // per-warp [da_s; da_d] partials
-  DevBuf anf[2], aef[2], acsr[2];   // occu_predict_async: double-buffered input staging
+  DevBuf anf[2], aef[2], acsr[2];   // occu_predict_async / occu_train_step_async: double-buffered input staging
+  DevBuf aty[2];           // occu_train_step_async: staged targets
   DevBuf dT, dZ;           // decoder readout: per-node FFN hidden / output rows [N][d]
   DevBuf dprep;            // decoder readout: folded key map M [d][16] and offsets c [16]
   DevBuf dpool;            // decoder readout: pool partials [B][8][16·d + 32]

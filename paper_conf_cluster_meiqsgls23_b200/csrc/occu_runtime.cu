@@ -50,7 +50,7 @@ void Workspace::release_all() {
   DevBuf *bufs[] = {&node_feat, &edge_feat, &targets, &out_occ, &csr, &e0, &g, &r, &c, &yhat,
                     &dy, &dc, &dr, &dh, &dhprev, &dP, &MG, &DV, &DZ, &deA, &deB, &dalpha,
                     &dpq, &partial, &loss, &tcpart, &dpart, &rpart, &anf[0], &anf[1],
-                    &aef[0], &aef[1], &acsr[0], &acsr[1], &dT, &dZ, &dprep, &dpool, &gx, &gqkv, &go, &gscr, &gdh[0], &gdh[1], &dbwd, &hub,
+                    &aef[0], &aef[1], &acsr[0], &acsr[1], &dT, &dZ, &dprep, &dpool, &gx, &gqkv, &go, &gscr, &gdh[0], &gdh[1], &dbwd, &hub, &aty[0], &aty[1],
                     &scsr, &snf, &sef, &sdesc, &hf};
   for (DevBuf *b : bufs) b->release();
   for (auto *v : {&hbar, &p, &q, &e, &h, &gs, &gh, &gsave})
@@ -416,8 +416,7 @@ occu_status check_ready(occu_ctx *ctx) {
   return OCCU_OK;
 }
 
-occu_status grads_impl(occu_ctx *ctx, const occu_batch *batch, const float *targets, Staged &stg,
-                       DevCsr &csr) {
+occu_status check_train(occu_ctx *ctx, const occu_batch *batch, const float *targets) {
   occu_status st = check_ready(ctx);
   if (st != OCCU_OK) return st;
   if (!batch || !batch->csr || !targets) return fail(ctx, OCCU_EINVAL, "batch/targets NULL");
@@ -428,10 +427,14 @@ occu_status grads_impl(occu_ctx *ctx, const occu_batch *batch, const float *targ
     return fail(ctx, OCCU_EINVAL, "training through the Graphormer layers / decoder readout runs in OCCU_FP32 on kernel path 0");
   if (ctx->cfg.msg == OCCU_MSG_NEIGHBOR_SOFTMAX && ctx->cfg.prec == OCCU_BF16)
     return fail(ctx, OCCU_EINVAL, "reading B in OCCU_BF16 is inference-only in this build");
-  ctx->launches = 0;
-  if ((st = resolve_csr(ctx, batch->csr, csr)) != OCCU_OK) return st;
-  if ((st = stage_inputs(ctx, csr, batch->node_feat, batch->edge_feat, targets, stg)) != OCCU_OK)
-    return st;
+  return OCCU_OK;
+}
+
+// Forward with saves + backward of a batch already on the device (csr, stg device pointers);
+// gradients (+ the loss in slot `total`) land in ctx->grads.
+occu_status grads_core(occu_ctx *ctx, const DevCsr &csr, const Staged &stg, int32_t global_B) {
+  occu_status st;
+  const bool stack = ctx->cfg.readout == OCCU_READOUT_SET_DECODER || ctx->cfg.graphormer > 0;
   if ((st = forward(ctx, csr, stg.nf, stg.ef, true)) != OCCU_OK) return st;
   const occu_config &c = ctx->cfg;
   const ParamLayout &L = ctx->layout;
@@ -451,7 +454,7 @@ occu_status grads_impl(occu_ctx *ctx, const occu_batch *batch, const float *targ
   CK(w.dpq.ensure(size_t(csr.N) * 8), "alloc");
   CK(w.loss.ensure(4), "alloc");
   cudaStream_t s = ctx->stream;
-  LK(launch_head_backward(ctx, csr, stg.y, batch->global_num_graphs, s), "head backward");
+  LK(launch_head_backward(ctx, csr, stg.y, global_B, s), "head backward");
   if (stack) {
     // NEXT-2 / NEXT-3 training: ∂L/∂(stack top) from the readout, then the Graphormer layers in
     // reverse, then dA of the last ANEE layer (what the ANEE backward consumes in w.dh)
@@ -505,6 +508,16 @@ occu_status grads_impl(occu_ctx *ctx, const occu_batch *batch, const float *targ
   return OCCU_OK;
 }
 
+occu_status grads_impl(occu_ctx *ctx, const occu_batch *batch, const float *targets, Staged &stg,
+                       DevCsr &csr) {
+  occu_status st = check_train(ctx, batch, targets);
+  if (st != OCCU_OK) return st;
+  ctx->launches = 0;
+  if ((st = resolve_csr(ctx, batch->csr, csr)) != OCCU_OK) return st;
+  if ((st = stage_inputs(ctx, csr, batch->node_feat, batch->edge_feat, targets, stg)) != OCCU_OK)
+    return st;
+  return grads_core(ctx, csr, stg, batch->global_num_graphs);
+}
 
 // ---- NCCL watchdog -------------------------------------------------------------------
 // The communicator is non-blocking (ncclConfig_t::blocking = 0): NCCL calls return at once
@@ -559,6 +572,25 @@ occu_status stream_wait(occu_ctx *ctx, const char *what) {
       return nccl_abort(ctx, std::string(what) + ": no progress within the timeout (ncclCommAbort)");
     usleep(20);
   }
+}
+
+// a11 + a12 after the backward: the NCCL allreduce (when a communicator exists), then Adam.
+occu_status allreduce_adam(occu_ctx *ctx, float lr) {
+  occu_status st;
+  const size_t n = ctx->layout.total + 1;
+  if (ctx->comm_aborted && !ctx->comm)
+    return fail(ctx, OCCU_ENCCL, "the communicator was aborted; call occu_dist_init again");
+  if (ctx->comm) {
+    // a11: sum of the flat gradient (+ loss slot) over the ranks, in place, on the ctx stream
+    ncclResult_t r = ncclAllReduce(ctx->grads.ptr, ctx->grads.ptr, n, ncclFloat32, ncclSum,
+                                   ctx->comm, ctx->stream);
+    if (r != ncclSuccess && r != ncclInProgress)
+      return nccl_abort(ctx, std::string("ncclAllReduce: ") + ncclGetErrorString(r));
+    if ((st = nccl_settle(ctx, "ncclAllReduce")) != OCCU_OK) return st;
+  }
+  ctx->adam_t += 1;
+  LK(launch_adam(ctx, lr, ctx->stream), "adam");
+  return OCCU_OK;
 }
 
 }  // namespace
@@ -828,19 +860,7 @@ occu_status occu_train_step(occu_ctx *ctx, const occu_batch *batch, const float 
   DevCsr csr;
   occu_status st = grads_impl(ctx, batch, targets, stg, csr);
   if (st != OCCU_OK) return st;
-  const size_t n = ctx->layout.total + 1;
-  if (ctx->comm_aborted && !ctx->comm)
-    return fail(ctx, OCCU_ENCCL, "the communicator was aborted; call occu_dist_init again");
-  if (ctx->comm) {
-    // a11: sum of the flat gradient (+ loss slot) over the ranks, in place, on the ctx stream
-    ncclResult_t r = ncclAllReduce(ctx->grads.ptr, ctx->grads.ptr, n, ncclFloat32, ncclSum,
-                                   ctx->comm, ctx->stream);
-    if (r != ncclSuccess && r != ncclInProgress)
-      return nccl_abort(ctx, std::string("ncclAllReduce: ") + ncclGetErrorString(r));
-    if ((st = nccl_settle(ctx, "ncclAllReduce")) != OCCU_OK) return st;
-  }
-  ctx->adam_t += 1;
-  LK(launch_adam(ctx, lr, ctx->stream), "adam");
+  if ((st = allreduce_adam(ctx, lr)) != OCCU_OK) return st;
   if (out_loss || stg.host) {
     float l = 0.f;
     CK(cudaMemcpyAsync(&l, ctx->grads.as<float>() + ctx->layout.total, 4, cudaMemcpyDeviceToHost,
@@ -848,6 +868,59 @@ occu_status occu_train_step(occu_ctx *ctx, const occu_batch *batch, const float 
     if ((st = stream_wait(ctx, "train step")) != OCCU_OK) return st;
     if (out_loss) *out_loss = l;
   }
+  return OCCU_OK;
+}
+
+occu_status occu_train_step_async(occu_ctx *ctx, const occu_batch *batch, const float *targets,
+                                  float lr, float *out_loss) {
+  occu_status st = check_train(ctx, batch, targets);
+  if (st != OCCU_OK) return st;
+  const occu_csr_batch *hb = batch->csr;
+  if (hb->on_device || !batch->node_feat || is_device_ptr(batch->node_feat) || is_device_ptr(targets) ||
+      (out_loss && is_device_ptr(out_loss)) || (hb->num_edges > 0 && !batch->edge_feat))
+    return fail(ctx, OCCU_EINVAL, "occu_train_step_async takes a host batch and host (pinned) buffers");
+  if (!ctx->copy_stream) {
+    CK(cudaStreamCreateWithFlags(&ctx->copy_stream, cudaStreamNonBlocking), "copy stream");
+    for (int k = 0; k < 2; ++k) {
+      CK(cudaEventCreateWithFlags(&ctx->a_copied[k], cudaEventDisableTiming), "event");
+      CK(cudaEventCreateWithFlags(&ctx->a_free[k], cudaEventDisableTiming), "event");
+    }
+  }
+  ctx->launches = 0;
+  const int slot = ctx->a_slot;
+  ctx->a_slot ^= 1;
+  // the previous call's host inputs become reusable once its copies have landed
+  CK(cudaEventSynchronize(ctx->a_copied[slot ^ 1]), "wait previous copy");
+  const occu_config &c = ctx->cfg;
+  Workspace &w = ctx->ws;
+  // the slot's buffers are reused only after the step that read them has finished
+  CK(cudaStreamWaitEvent(ctx->copy_stream, ctx->a_free[slot], 0), "wait slot");
+  DevCsr csr;
+  if ((st = upload_csr(ctx, hb, w.acsr[slot], ctx->copy_stream, csr)) != OCCU_OK) return st;
+  CK(w.anf[slot].ensure(size_t(csr.N) * c.F_n * 4), "alloc node_feat");
+  CK(w.aef[slot].ensure(std::max<size_t>(size_t(csr.E) * c.F_e * 4, 4)), "alloc edge_feat");
+  CK(w.aty[slot].ensure(size_t(csr.B) * 4), "alloc targets");
+  CK(cudaMemcpyAsync(w.anf[slot].ptr, batch->node_feat, size_t(csr.N) * c.F_n * 4,
+                     cudaMemcpyHostToDevice, ctx->copy_stream), "node_feat H2D");
+  if (csr.E > 0)
+    CK(cudaMemcpyAsync(w.aef[slot].ptr, batch->edge_feat, size_t(csr.E) * c.F_e * 4,
+                       cudaMemcpyHostToDevice, ctx->copy_stream), "edge_feat H2D");
+  CK(cudaMemcpyAsync(w.aty[slot].ptr, targets, size_t(csr.B) * 4, cudaMemcpyHostToDevice,
+                     ctx->copy_stream), "targets H2D");
+  CK(cudaEventRecord(ctx->a_copied[slot], ctx->copy_stream), "record");
+  CK(cudaStreamWaitEvent(ctx->stream, ctx->a_copied[slot], 0), "wait copy");
+  Staged stg;
+  stg.nf = w.anf[slot].as<float>();
+  stg.ef = w.aef[slot].as<float>();
+  stg.y = w.aty[slot].as<float>();
+  stg.host = false;
+  if ((st = grads_core(ctx, csr, stg, batch->global_num_graphs)) != OCCU_OK) return st;
+  if ((st = allreduce_adam(ctx, lr)) != OCCU_OK) return st;
+  CK(cudaEventRecord(ctx->a_free[slot], ctx->stream), "record");
+  if (out_loss)
+    CK(cudaMemcpyAsync(out_loss, ctx->grads.as<float>() + ctx->layout.total, 4,
+                       cudaMemcpyDeviceToHost, ctx->stream), "loss D2H");
+  CK(cudaGetLastError(), "train_step_async");
   return OCCU_OK;
 }
 

@@ -33,7 +33,7 @@ EXPORTS = [
     "occu_get_tensor", "occu_last_launch_count", "occu_last_error", "occu_set_profiling",
     "occu_profile_reset", "occu_profile_query", "occu_set_kernel_path", "occu_pack_jobs",
     "occu_template_create", "occu_template_destroy", "occu_synthesize", "occu_set_small_batch_kernel",
-    "occu_dist_set_timeout", "occu_dist_abort", "occu_dist_sync",
+    "occu_dist_set_timeout", "occu_dist_abort", "occu_dist_sync", "occu_train_step_async",
 ]
 
 
@@ -102,6 +102,7 @@ def lib():
             "occu_predict_async": ([VP, P(CsrBatch), VP, VP, VP], I32),
             "occu_wait": ([VP], I32),
             "occu_train_step": ([VP, P(BatchStruct), VP, C.c_float, P(C.c_float)], I32),
+            "occu_train_step_async": ([VP, P(BatchStruct), VP, C.c_float, VP], I32),
             "occu_compute_grads": ([VP, P(BatchStruct), VP, P(C.c_float)], I32),
             "occu_get_grads": ([VP, VP, SZ], I32),
             "occu_set_weight_decay": ([VP, C.c_float], I32),
@@ -468,6 +469,18 @@ class Model:
         _check(lib().occu_train_step(self._ctx, C.byref(b), tp, lr,
                                      C.byref(loss) if want_loss else None), self._ctx)
         return float(loss.value) if want_loss else None
+
+    def train_step_async(self, csr: Csr, node_feat, edge_feat, targets, lr: float,
+                         global_num_graphs=None, out_loss=None):
+        """occu_train_step_async: host batch, pinned host features / targets; returns at once.
+        out_loss: optional pinned 1-element float32 tensor, valid after wait().  The arguments
+        stay referenced until the next call (inputs) or wait() (out_loss)."""
+        b, keep = self._batch(csr, node_feat, edge_feat, global_num_graphs)
+        tp, _, k3 = _ptr(targets)
+        lp = out_loss.data_ptr() if out_loss is not None else None
+        _check(lib().occu_train_step_async(self._ctx, C.byref(b), tp, lr, lp), self._ctx)
+        self._inflight = ([(None, None, None, None, None, None, x[6]) for x in self._inflight]
+                          + [(csr, keep, k3, b, node_feat, edge_feat, out_loss)])
 
     def compute_grads(self, csr: Csr, node_feat, edge_feat, targets, global_num_graphs=None):
         b, keep = self._batch(csr, node_feat, edge_feat, global_num_graphs)

@@ -539,3 +539,30 @@ def test_hub_path_matches_oracle_and_is_deterministic(prec):
             got = m.get_tensor(occu.T_H, i, (pk["num_nodes"], c.d))
             assert rel(got, ref["layers"][i]["h"]) <= TOL
             rows_ok(got, ref["layers"][i]["h"], TOL, ("h", i))
+
+
+def test_train_step_async_matches_blocking_bitwise():
+    """occu_train_step_async (pinned host inputs, copies on the copy stream, double-buffered
+    staging) over a stream of different batches: parameters and losses bitwise equal to the
+    blocking occu_train_step sequence; device inputs are rejected."""
+    import torch
+    c = mk(2, 64)
+    batches = [configs.random_dag_batch(20 + 5 * k, 1400 + k, max_nodes=50, hub=True) for k in range(4)]
+    flat = weights.unit_scale(wcfg(c), weights.init_flat(wcfg(c), 17))
+    ms, ma = occu.Model(c), occu.Model(c)
+    ms.set_params(flat)
+    ma.set_params(flat)
+    want = [ms.train_step(occu.pack(b.graphs), b.node_feat, b.edge_feat, b.targets, 1e-3,
+                          global_num_graphs=64) for b in batches]
+    pins = [(torch.from_numpy(b.node_feat).pin_memory(), torch.from_numpy(b.edge_feat).pin_memory(),
+             torch.from_numpy(b.targets).pin_memory(), torch.zeros(1).pin_memory()) for b in batches]
+    for b, (nf, ef, y, lo) in zip(batches, pins):
+        ma.train_step_async(occu.pack(b.graphs), nf, ef, y, 1e-3, global_num_graphs=64, out_loss=lo)
+    ma.wait()
+    assert [float(p[3][0]) for p in pins] == want
+    assert np.array_equal(ma.get_params(), ms.get_params())
+    dev = torch.device("cuda", 0)
+    b = batches[0]
+    with pytest.raises(occu.OccuError):
+        ma.train_step_async(occu.pack(b.graphs), torch.from_numpy(b.node_feat).to(dev),
+                            torch.from_numpy(b.edge_feat).to(dev), torch.from_numpy(b.targets).to(dev), 1e-3)
