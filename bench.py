@@ -322,9 +322,22 @@ def cpu_baseline_sample(cfg3_batch, seconds=15.0):
                                       cfg3_batch.num_graphs)
         done += 1
     dt = time.perf_counter() - t0
-    return {"value": done / dt, "unit": "graphs/s", "cores": cpu_cores_used(), "kind": "oracle",
-            "sample": f"{done} CFG3 graphs (BERT-base / GPT-2, L=3, d=128), one float64 NumPy "
-                      f"oracle training step (fwd, MSE, bwd, Adam) per graph, {dt:.1f} s"}
+    out = {"value": done / dt, "unit": "graphs/s", "cores": cpu_cores_used(), "kind": "oracle",
+           "sample": f"{done} CFG3 graphs (BERT-base / GPT-2, L=3, d=128), one float64 NumPy "
+                     f"oracle training step (fwd, MSE, bwd, Adam) per graph, {dt:.1f} s"}
+    try:        # the same oracle restricted to one BLAS thread (SURVEY §8(d)'s single-thread figure)
+        from threadpoolctl import threadpool_limits
+        with threadpool_limits(limits=1):
+            done1, t1 = 0, time.perf_counter()
+            while time.perf_counter() - t1 < seconds / 3:
+                i = (done1 // 2) % half + (half if done1 % 2 else 0)
+                params, _ = oracle_train_step(oracle, ocf, params, state, cfg3_batch.subset([i]),
+                                              cfg3_batch.num_graphs)
+                done1 += 1
+            out["single_thread_value"] = done1 / (time.perf_counter() - t1)
+    except Exception:                                   # noqa: BLE001 — optional figure
+        pass
+    return out
 
 
 # ---------------------------------------------------------------- the GPU bench

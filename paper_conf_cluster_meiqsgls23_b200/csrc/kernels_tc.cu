@@ -15,17 +15,19 @@
 // accumulates x0·w0 + x0·w1 + x1·w0 in FP32 (TMEM); the dropped x1·w1 term is
 // ~2^-22 relative.  The epilogue multiplies by 2^-(e_r + f), which is exact.
 //
-// CTA = 6 warps, persistent over 128-row tiles, 1 CTA per SM:
-//   warp 0     producer: per-row cp.async.bulk of the next tiles into a 2-slot
-//              ring of padded fp32 row buffers (mbarrier complete_tx);
-//   warp 1     TMEM allocator + MMA issuer: 3·K/16 tcgen05.mma (M=128, N=D,
-//              K=16, A from TMEM, B = SW128 K-major weight images in smem),
-//              commit -> accumulator-full / A-free mbarriers;
-//   warps 2-5  workers, thread = row: split their row into TMEM A[i%2]
-//              (tcgen05.st), then run the epilogue of the previous tile from
-//              the TMEM accumulator ACC[(i-1)%2] (tcgen05.ld).
-// TMEM: A[2] x 128 columns + ACC[2] x 128 columns = 512.  Loads of tile i+1,
-// the MMAs of tile i and the epilogue of tile i-1 overlap.
+// CTA = 26 warps (NTH = 832), persistent over 128-row tiles, 1 CTA per SM:
+//   warp 0       producer: bulk copy of the weight images, then 2D TMA loads (128 rows x 32
+//                fp32 SW128 boxes, OOB rows zero-filled) of the next tiles into a 2-slot ring;
+//   warp 1       TMEM allocator + MMA issuer: 3·K/16 tcgen05.mma (M=128, N=D, K=16, A from
+//                TMEM, B = SW128 K-major weight images in smem), commit -> accumulator-full /
+//                A-free mbarriers;
+//   warps 2-9    converters, thread = (row, K-half): per-row power-of-two scale (row max
+//                exchanged between the halves), fp16x2 split into TMEM A[i%2] (tcgen05.st);
+//   warps 10-25  epilogue, two groups of 8 warps on alternating tiles (two warps per TMEM lane
+//                quarter, one per column half): tcgen05.ld of ACC[i%2], the fused row epilogue,
+//                coalesced stores through per-warp transpose buffers.
+// TMEM: A[2] x 128 columns + ACC[2] x 128 columns = 512.  Loads of tile i+1, the MMAs of
+// tile i and the epilogues of tiles i-1, i-2 overlap.
 #include <cuda_bf16.h>
 #include <cuda_fp16.h>
 #include <cuda_runtime.h>
