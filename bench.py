@@ -42,7 +42,7 @@ import numpy as np  # noqa: E402
 
 L2_BYTES = 126 * 1024 * 1024
 LR = 1e-4                      # P273: Adam, lr = 1e-4
-ALL_SECTIONS = ["cfg3_bf16", "cfg2", "cfg2_train", "micro", "readingb", "decoder", "graphormer",
+ALL_SECTIONS = ["cfg3_bf16", "cfg2", "cfg2_paper", "cfg2_train", "micro", "readingb", "decoder", "graphormer",
                 "paper_stack", "paper_stack_train", "cfg1", "cfg4", "cfg5"]
 METRIC = "GNN graphs/sec (train & infer) at 1/2/4/8 B200; aggregation HBM GB/s vs peak"
 
@@ -504,6 +504,17 @@ class Bench:
         tot_alg = sum(v for k, v in alg.items() if k in prof)
         loss_after = m.train_step(csr, nf, ef, yt, LR, global_num_graphs=gB)
 
+        if a.no_e2e:                # profiling runs (ncu launch list): the device step only
+            e2e = {"value": None, "unit": "graphs/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0,
+                   "ms_per_step": None, "skipped": "--no-e2e"}
+            self.details["cfg3_f32"] = {"kernels": kernels, "roofline": roof, "loss_first": loss0,
+                                        "loss_after": loss_after, "clocks": clocks}
+            del nf, ef, yt, csr, m
+            torch.cuda.empty_cache()
+            return {"B": B, "N": N, "E": E, "gB": gB, "ms": ms, "launches": launches,
+                    "roof": roof, "clocks": clocks, "e2e": e2e, "loss0": loss0,
+                    "loss_after": loss_after,
+                    "step_frac": tot_alg / (ms * 1e-3) / 1e9 / self.peaks["hbm_gbs"]}
         # e2e through the public API: per step occu_pack of the batch's edge lists (host C++),
         # occu_train_step with pinned HOST buffers (CSR + features + targets H2D inside the
         # call), the loss read back D2H (the call returns it)
@@ -643,6 +654,34 @@ class Bench:
                 if prec == occu.FP32:
                     self.aggregation = agg
             del m, csr
+
+    def sec_cfg2_paper(self):
+        """the paper's encoder shape (L = 1, d = 256; P273 "hidden
+        dimension of all the layers to 256") on CFG2's 256 ResNet-50 graphs, FP32 inference on
+        the CTA-pair tensor-core path (tcgen05.mma.cta_group::2, kernels_tc.cu)."""
+        b = self._cfg2()
+        _, nf, ef, _ = self.cfg2_dev
+        B, N, E, d = b.num_graphs, b.num_nodes, b.num_edges, 256
+        m = self.model(L=1, d=d)
+        m.init_weights(42)
+        csr = m.to_device(self.cfg2_host_csr)
+        alg = algorithmic_bytes(N, E, B, d=d, L=1, rrows=readout_rows(b.graphs))
+        ms, prof, _ = self._infer("cfg2_paper_f32", m, csr, nf, ef, B, alg, "f32")
+        det = self.details["cfg2_paper_f32"]
+        sv = survey_step_bytes(N, E, B, d=d, L=1)
+        det["survey_step_bytes"] = sv
+        det["step_frac_of_hbm_survey_bytes"] = sv / (ms * 1e-3) / 1e9 / self.peaks["hbm_gbs"]
+        if "gate_tc" in prof:          # the dense contraction W_m e' (E x 256 x 256)
+            ams = prof["gate_tc"][0] / self.args.steps
+            flops = 2.0 * E * d * d
+            peak = self.peaks["bf16_tflops"] / 3.0
+            det["gate_tensor_roofline"] = {
+                "kernel": "gate_tc (rowgemm_pair_kernel)", "bound": "tensor",
+                "achieved": flops / (ams * 1e-3) / 1e12, "peak": peak, "unit": "TFLOP/s",
+                "frac": flops / (ams * 1e-3) / 1e12 / peak,
+                "peak_kind": "measured bf16 dense (= fp16 kind::f16) / 3 products (fp16x2 split)"}
+        det["bf16"] = "unavailable: d = 256 runs OCCU_FP32 only in this build"
+        del m, csr
 
     def sec_cfg2_train(self):
         occu, torch = self.occu, self.torch
@@ -1051,8 +1090,8 @@ class Bench:
         roof_c = {k: roof.get(k) for k in ("kernel", "bound", "achieved", "peak", "unit", "frac",
                                             "traffic", "algorithmic_bytes_per_launch",
                                             "avg_launch_ms", "share_of_step", "peak_kind")}
-        e2e = {k: hl["e2e"][k] for k in ("value", "unit", "ms_per_step", "h2d_bytes_per_step",
-                                          "d2h_bytes_per_step")}
+        e2e = {k: hl["e2e"].get(k) for k in ("value", "unit", "ms_per_step", "h2d_bytes_per_step",
+                                              "d2h_bytes_per_step")}
         line = {
             "metric": METRIC, "value": value, "unit": "graphs/s", "n_gpus": self.world,
             "steps": a.steps, "warmup": a.warmup, "ms_per_step": hl["ms"],
@@ -1103,6 +1142,7 @@ def parse(argv=None):
     ap.add_argument("--ref-graphs", type=int, default=1)
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--no-flush", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true", help="skip the e2e legs (profiling runs only)")
     args = ap.parse_args(argv)
     if args.warmup < 3:
         args.warmup = 3

@@ -289,6 +289,9 @@ template <int V>
 __device__ __forceinline__ void store_row(float *dst, const float (&v)[V]) {
   if constexpr (V == 4) {
     *reinterpret_cast<float4 *>(dst) = make_float4(v[0], v[1], v[2], v[3]);
+  } else if constexpr (V == 8) {
+    *reinterpret_cast<float4 *>(dst) = make_float4(v[0], v[1], v[2], v[3]);
+    *reinterpret_cast<float4 *>(dst + 4) = make_float4(v[4 % V], v[5 % V], v[6 % V], v[7 % V]);
   } else {
 #pragma unroll
     for (int c = 0; c < V; ++c) dst[c] = v[c];
@@ -429,6 +432,11 @@ __device__ __forceinline__ void load_row(const void *base, long row, int D, int 
     if constexpr (V == 4) {
       const float4 a = __ldg(reinterpret_cast<const float4 *>(p));
       v[0] = a.x; v[1 % V] = a.y; v[2 % V] = a.z; v[3 % V] = a.w;
+    } else if constexpr (V == 8) {
+      const float4 a = __ldg(reinterpret_cast<const float4 *>(p));
+      const float4 b = __ldg(reinterpret_cast<const float4 *>(p + 4));
+      v[0] = a.x; v[1 % V] = a.y; v[2 % V] = a.z; v[3 % V] = a.w;
+      v[4 % V] = b.x; v[5 % V] = b.y; v[6 % V] = b.z; v[7 % V] = b.w;
     } else {
 #pragma unroll
       for (int c = 0; c < V; ++c) v[c] = __ldg(p + c);
@@ -444,6 +452,33 @@ template <> struct RawRow<4, false> {
     v = __ldg(reinterpret_cast<const float4 *>(reinterpret_cast<const float *>(b) + row * D + lane * 4));
   }
   __device__ __forceinline__ void get(float (&o)[4]) const { o[0] = v.x; o[1] = v.y; o[2] = v.z; o[3] = v.w; }
+};
+// d = 256: a lane's 8 channels = two float4 (one 1 KB row per warp, fully coalesced)
+template <> struct RawRow<8, false> {
+  float4 v0, v1;
+  __device__ __forceinline__ void load(const void *b, long row, int D, int lane) {
+    const float4 *p = reinterpret_cast<const float4 *>(reinterpret_cast<const float *>(b) + row * D + lane * 8);
+    v0 = __ldg(p);
+    v1 = __ldg(p + 1);
+  }
+  __device__ __forceinline__ void get(float (&o)[8]) const {
+    o[0] = v0.x; o[1] = v0.y; o[2] = v0.z; o[3] = v0.w;
+    o[4] = v1.x; o[5] = v1.y; o[6] = v1.z; o[7] = v1.w;
+  }
+};
+template <> struct RawRow<8, true> {
+  uint4 v;
+  __device__ __forceinline__ void load(const void *b, long row, int D, int lane) {
+    v = __ldg(reinterpret_cast<const uint4 *>(reinterpret_cast<const __nv_bfloat16 *>(b) + row * D + lane * 8));
+  }
+  __device__ __forceinline__ void get(float (&o)[8]) const {
+    const uint32_t w[4] = {v.x, v.y, v.z, v.w};
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+      o[2 * i] = __uint_as_float(w[i] << 16);
+      o[2 * i + 1] = __uint_as_float(w[i] & 0xFFFF0000u);
+    }
+  }
 };
 template <> struct RawRow<2, false> {
   float2 v;
@@ -482,7 +517,8 @@ __device__ __forceinline__ void store_row_t(void *base, long row, int D, int lan
       const __nv_bfloat162 h = __floats2bfloat162_rn(v[c], v[c + 1]);
       w[c / 2] = *reinterpret_cast<const uint32_t *>(&h);
     }
-    if constexpr (V == 4) *reinterpret_cast<uint2 *>(p) = make_uint2(w[0], w[1]);
+    if constexpr (V == 8) *reinterpret_cast<uint4 *>(p) = make_uint4(w[0], w[1 % (V / 2)], w[2 % (V / 2)], w[3 % (V / 2)]);
+    else if constexpr (V == 4) *reinterpret_cast<uint2 *>(p) = make_uint2(w[0], w[1 % (V / 2)]);
     else *reinterpret_cast<uint32_t *>(p) = w[0];
   } else {
     store_row<V>(reinterpret_cast<float *>(base) + row * D + lane * V, v);
@@ -1940,7 +1976,12 @@ static int gather_impl(const occu_ctx *ctx, const DevCsr &csr, const float *g, c
   if (r0 < 0) return r0;
   OCCU_PROF_BEGIN(ctx, "gather_segsum", st);
 #define OCCU_GATHER_ARGS g, hbar, csr.in_ptr, csr.in_src, csr.N, mean, ctx->cfg.slope, h_out, csr.node_graph, rpart, hub, csr.in_dst
-  if (variant == 0) {
+  if constexpr (D == 256) {
+    // d = 256: two (g, h̄) row pairs in flight per lane (16 floats each); 1 KB rows
+    const int grid = grid_for(long(csr.N) * 4, NT, occ * ctx->num_sms);
+    if (rpart) launch_pdl(ctx->pdl & 2, gather_segsum_v2_kernel<D, 2, true>, grid, NT, 0, st, OCCU_GATHER_ARGS);
+    else launch_pdl(ctx->pdl & 2, gather_segsum_v2_kernel<D, 2, false>, grid, NT, 0, st, OCCU_GATHER_ARGS);
+  } else if (variant == 0) {
     const int grid = grid_for(long(csr.N) * 4, NT, 16 * ctx->num_sms);
 #define OCCU_GATHER_ARGS0 g, hbar, csr.in_ptr, csr.in_src, csr.N, mean, ctx->cfg.slope, h_out, csr.node_graph, rpart
     if (rpart) gather_segsum_kernel<D, true><<<grid, NT, 0, st>>>(OCCU_GATHER_ARGS0);
@@ -2057,6 +2098,7 @@ int launch_gather_segsum(const occu_ctx *ctx, const DevCsr &csr, const float *g,
   switch (ctx->cfg.d) {
     case 64: return gather_impl<64>(ctx, csr, g, hbar, h_out, rpart, st);
     case 128: return gather_impl<128>(ctx, csr, g, hbar, h_out, rpart, st);
+    case 256: return gather_impl<256>(ctx, csr, g, hbar, h_out, rpart, st);
     default: return -int(cudaErrorInvalidValue);
   }
 }
@@ -2090,7 +2132,8 @@ int launch_readout_head(const occu_ctx *ctx, const DevCsr &csr, const float *h, 
 #define OCCU_RO_ARGS h, csr.node_off, cf.d_h, params + L.W_1, params + L.b_1, params + L.w_2, \
     params + L.b_2, cf.slope, r, c, yhat, chunked ? 8 : 0
   if (cf.d == 64) launch_pdl(ctx->pdl & 8, readout_head_kernel<64>, csr.B, RO_WARPS * 32, smem, st, OCCU_RO_ARGS);
-  else launch_pdl(ctx->pdl & 8, readout_head_kernel<128>, csr.B, RO_WARPS * 32, smem, st, OCCU_RO_ARGS);
+  else if (cf.d == 128) launch_pdl(ctx->pdl & 8, readout_head_kernel<128>, csr.B, RO_WARPS * 32, smem, st, OCCU_RO_ARGS);
+  else launch_pdl(ctx->pdl & 8, readout_head_kernel<256>, csr.B, RO_WARPS * 32, smem, st, OCCU_RO_ARGS);
 #undef OCCU_RO_ARGS
   OCCU_PROF_END(ctx);
   LAUNCH_CHECK();

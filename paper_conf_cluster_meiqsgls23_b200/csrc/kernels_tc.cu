@@ -868,6 +868,378 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
 }
 
 // ---------------------------------------------------------------------------
+// d = 256, the paper's hidden width (P273 "hidden dimension of all the layers to 256"):
+// the same three forward row-GEMMs (EPI_NODE / EPI_EDGE / EPI_GATE, same fused epilogues and
+// fp16x2 split as rowgemm_kernel) on a CTA PAIR.  One CTA cannot hold the fp16x2 images of
+// a 256 x 256 matrix (2 x 128 KB > 227 KB of shared memory), so two CTAs of a cluster on
+// neighbouring SMs run tcgen05.mma.cta_group::2: M = 256 rows per MMA (128 per CTA, A and
+// the accumulator in each CTA's own TMEM), B split along N (each CTA keeps the images of
+// its 128 output channels, resident for the whole kernel).  Each CTA ends up with full
+// 256-channel rows in TMEM, so the row epilogues (p/q dots, channel softmax) need no
+// exchange between the CTAs.
+//   warp 0      producer: the CTA's N-half of the images (bulk copies), then 2D TMA boxes
+//               (128 rows x 32 fp32, SW128) of its rows into a P_NS-box ring;
+//   warp 1      TMEM (512 columns, cta_group::2 alloc in both CTAs); in the leader CTA the
+//               MMA issuer: 3·K/16 tcgen05.mma.cta_group::2 (M=256, N=256, K=16) per pair
+//               tile, committed to BOTH CTAs' barriers (multicast);
+//   warps 2-9   converters, thread = (row, box parity): fp16x2 split of each box into TMEM
+//               A (hi [0, Kpad/2), lo [Kpad/2, Kpad)); node inputs get the per-row power-of-two
+//               scale from the row max, read once from global memory (L2-resident for the
+//               TMA reads that follow); then one arrive per warp on the LEADER's A-full;
+//   warps 10-25 epilogue, thread = (row, 64-channel quarter): tcgen05.ld of the 256-column
+//               accumulator, the row epilogue (quarters combined in fixed order through
+//               shared memory), coalesced stores; one arrive per warp on the leader's
+//               accumulator-free barrier.
+// TMEM per CTA: A [0, 256) + ACC [256, 512), single-buffered: the converters of tile i+1 run
+// during the epilogue of tile i.  Pair tile t covers rows [256t, 256t + 256): rows
+// [256t + 128·rank, +128) live in CTA `rank`.
+// ---------------------------------------------------------------------------
+constexpr int P_NTH = 832;
+constexpr int P_NS = 4;               // input ring depth (boxes of 16 KB)
+constexpr int PD = 256;
+
+struct PairSmem {
+  uint8_t *w0, *w1;                   // this CTA's N-half of [w0 | w1]: [Kpad/64][128 rows][128 B]
+  float *ring;                        // P_NS x 4096 floats
+  uint64_t *full, *empty;             // [P_NS]
+  uint64_t *afull, *afree, *accfull, *accfree, *wfull, *wpeer, *eready;
+  uint32_t *tmem_slot;
+  float *avec;                        // [2][256] a_s, a_d (NODE)
+  int *erow;                          // [4][128]
+  float *cmax;                        // [2][128]
+  float *xch;                         // [2 values][4 quarters][128 rows]
+  float *xbuf;                        // 16 epilogue warps x 16 x 20 floats
+};
+
+__host__ __device__ inline size_t pair_smem_bytes(int K) {
+  const size_t img = size_t(kpad_of(K)) * 128 * 2;
+  return 1024 + 2 * img + size_t(P_NS) * 16384 + 256 + 2048 + 2048 + 1024 + 4096 + 16 * 16 * 20 * 4;
+}
+
+__device__ __forceinline__ PairSmem carve_pair(uint8_t *raw, int K) {
+  PairSmem s;
+  const uint32_t a = tc::smem_u32(raw);
+  uint8_t *base = raw + ((1024 - (a & 1023)) & 1023);
+  const size_t img = size_t(kpad_of(K)) * 128 * 2;
+  s.w0 = base;
+  s.w1 = base + img;
+  s.ring = reinterpret_cast<float *>(base + 2 * img);
+  uint8_t *misc = base + 2 * img + size_t(P_NS) * 16384;
+  uint64_t *bars = reinterpret_cast<uint64_t *>(misc);
+  s.full = bars;
+  s.empty = bars + P_NS;
+  s.afull = bars + 2 * P_NS;
+  s.afree = s.afull + 1;
+  s.accfull = s.afull + 2;
+  s.accfree = s.afull + 3;
+  s.wfull = s.afull + 4;
+  s.wpeer = s.afull + 5;
+  s.eready = s.afull + 6;             // 4
+  s.tmem_slot = reinterpret_cast<uint32_t *>(misc + 224);
+  s.avec = reinterpret_cast<float *>(misc + 256);
+  s.erow = reinterpret_cast<int *>(misc + 256 + 2048);
+  s.cmax = reinterpret_cast<float *>(misc + 256 + 4096);
+  s.xch = reinterpret_cast<float *>(misc + 256 + 4096 + 1024);
+  s.xbuf = reinterpret_cast<float *>(misc + 256 + 4096 + 1024 + 4096);
+  return s;
+}
+
+__device__ __forceinline__ void epi_bar_pair() { asm volatile("bar.sync 1, 512;" ::: "memory"); }
+
+template <int EPI>
+__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(P_NTH, 1)
+    rowgemm_pair_kernel(const __grid_constant__ CUtensorMap tmap, RowGemmArgs a) {
+  extern __shared__ uint8_t smem_raw[];
+  const int K = a.K, Kpad = kpad_of(K), NB = nbox_of(K);
+  PairSmem s = carve_pair(smem_raw, K);
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const uint32_t rank = tc::cluster_rank();
+
+  pdl_trigger();
+  if (threadIdx.x == 0) {
+    for (int j = 0; j < P_NS; ++j) {
+      tc::mbar_init(s.full + j, 1);
+      tc::mbar_init(s.empty + j, 128);
+    }
+    tc::mbar_init(s.afull, 16);       // 8 converter warps x 2 CTAs (leader's copy used)
+    tc::mbar_init(s.afree, 1);        // multicast commit
+    tc::mbar_init(s.accfull, 1);      // multicast commit
+    tc::mbar_init(s.accfree, 32);     // 16 epilogue warps x 2 CTAs (leader's copy used)
+    tc::mbar_init(s.wfull, 1);
+    tc::mbar_init(s.wpeer, 1);
+    for (int j = 0; j < 4; ++j) tc::mbar_init(s.eready + j, 256);
+    tc::fence_mbar_init();
+  }
+  if (warp == 1) tc::tmem_alloc2<TMEM_COLS>(s.tmem_slot);
+  pdl_wait();
+  const int fexp = __ldg(a.wfexp);
+  const bool noshift = __ldg(a.wfexp + 1) != 0;
+  if (EPI == EPI_NODE)
+    for (int i = threadIdx.x; i < PD; i += P_NTH) {
+      s.avec[i] = a.a_s[i];
+      s.avec[PD + i] = a.a_d[i];
+    }
+  tc::fence_before_sync();
+  __syncthreads();
+  tc::cluster_sync();                 // both CTAs: barriers initialised, TMEM allocated
+  tc::fence_after_sync();
+  const uint32_t tmem = *s.tmem_slot;
+
+  const int tiles = (a.R + 2 * TM - 1) / (2 * TM);
+  const int cid = int(tc::cluster_id_x()), ncl = int(tc::ncluster_x());
+  const int my = cid < tiles ? (tiles - 1 - cid) / ncl + 1 : 0;
+  auto row0_of = [&](int i) -> long {
+    int t = cid + i * ncl;
+    if (a.rev) t = tiles - 1 - t;
+    return long(t) * (2 * TM) + long(rank) * TM;
+  };
+
+  if (warp == 0) {
+    // ---------------- producer ----------------
+    if (lane == 0) {
+      tc::prefetch_tmap(&tmap);
+      const uint32_t ib = uint32_t(Kpad) * PD * 2;            // one full image (w0 or w1)
+      tc::mbar_arrive_expect_tx(s.wfull, uint32_t(Kpad) * 128u * 2u * 2u);
+      for (int c = 0; c < Kpad / 64; ++c) {                   // 16 KB per 64-wide K chunk
+        const uint32_t src = uint32_t(c) * 32768u + rank * 16384u;
+        tc::bulk_g2s(s.w0 + c * 16384, a.wimg + src, 16384, s.wfull);
+        tc::bulk_g2s(s.w1 + c * 16384, a.wimg + ib + src, 16384, s.wfull);
+      }
+      if (rank == 1) {                                       // tell the leader its B half is in
+        tc::mbar_wait(s.wfull, 0);
+        tc::mbar_arrive_cluster(s.wpeer, 0);
+      }
+      long q = 0;
+      for (int i = 0; i < my; ++i) {
+        const long r0 = row0_of(i);
+        for (int b = 0; b < NB; ++b, ++q) {
+          const int sl = int(q % P_NS);
+          if (q >= P_NS) tc::mbar_wait(s.empty + sl, uint32_t((q / P_NS) - 1) & 1u);
+          if (r0 < a.R) {
+            tc::mbar_arrive_expect_tx(s.full + sl, 16384u);
+            tc::tma_load_2d(s.ring + sl * 4096, &tmap, 32 * b, int(r0), s.full + sl);
+          } else {
+            tc::mbar_arrive(s.full + sl);                     // rows past R: nothing to load
+          }
+        }
+      }
+    }
+    __syncwarp();
+  } else if (warp == 1) {
+    // ---------------- MMA issuer (leader CTA) ----------------
+    if (rank == 0) {
+      const uint32_t idsc = tc::idesc(256, uint32_t(PD), tc::FMT_F16);
+      const uint32_t w0a = tc::smem_u32(s.w0), w1a = tc::smem_u32(s.w1);
+      const int nk = (K + 15) / 16;
+      tc::mbar_wait(s.wfull, 0);
+      tc::mbar_wait_cluster(s.wpeer, 0);
+      for (int i = 0; i < my; ++i) {
+        tc::mbar_wait_cluster(s.afull, uint32_t(i) & 1u);
+        if (i >= 1) tc::mbar_wait_cluster(s.accfree, uint32_t(i - 1) & 1u);
+        tc::fence_after_sync();
+        if (lane == 0) {
+          const uint32_t d = tmem + 256u;
+          for (int kk = 0; kk < nk; ++kk) {
+            const uint32_t boff = uint32_t(kk >> 2) * 16384u + uint32_t(kk & 3) * 32u;
+            const uint64_t b0 = tc::sdesc_sw128(w0a + boff), b1 = tc::sdesc_sw128(w1a + boff);
+            const uint32_t a0 = tmem + uint32_t(kk) * 8u;
+            const uint32_t a1 = a0 + uint32_t(Kpad / 2);
+            tc::mma2_f16_ts(d, a0, b0, idsc, kk > 0 ? 1u : 0u);
+            tc::mma2_f16_ts(d, a0, b1, idsc, 1u);
+            tc::mma2_f16_ts(d, a1, b0, idsc, 1u);
+          }
+          tc::mma2_commit_both(s.accfull);
+          tc::mma2_commit_both(s.afree);
+        }
+        __syncwarp();
+      }
+    }
+  } else if (warp < EPI0) {
+    // ---------------- converters: thread = (row, box parity) -> TMEM A ----------------
+    const int qd = warp & 3;
+    const int kh = (warp - 2) >> 2;
+    const int row = qd * 32 + lane;
+    const uint32_t lane_base = tmem + (uint32_t(qd * 32) << 16);
+    const int kmid = (K / 4 + 1) / 2 * 4;                     // row-max halves
+    for (int i = 0; i < my; ++i) {
+      const long r0 = row0_of(i);
+      const bool live = long(row) < a.R - r0;
+      if (i >= 1) tc::mbar_wait(s.afree, uint32_t(i - 1) & 1u);
+      int er = 0;                                              // e' in [0, 1]: unscaled
+      if (EPI == EPI_NODE) {
+        float mx = 0.f;
+        if (live) {
+          const float *src = a.A + (r0 + row) * K;
+          const int k0 = kh ? kmid : 0, k1 = kh ? K : kmid;
+#pragma unroll 4
+          for (int k = k0; k < k1; k += 4) {
+            const float4 v = __ldg(reinterpret_cast<const float4 *>(src + k));
+            mx = fmaxf(mx, fmaxf(fmaxf(fabsf(v.x), fabsf(v.y)), fmaxf(fabsf(v.z), fabsf(v.w))));
+          }
+        }
+        s.cmax[kh * 128 + row] = mx;
+        asm volatile("bar.sync 3, 256;" ::: "memory");
+        mx = fmaxf(mx, s.cmax[(kh ^ 1) * 128 + row]);
+        er = scale_exp(mx);
+        asm volatile("bar.sync 3, 256;" ::: "memory");
+      }
+      const float xs = ldexpf(1.f, er);
+      for (int b = kh; b < NB; b += 2) {
+        const long q = long(i) * NB + b;
+        const int sl = int(q % P_NS);
+        tc::mbar_wait(s.full + sl, uint32_t(q / P_NS) & 1u);
+        const float *box = s.ring + sl * 4096;
+        uint32_t x0[16], x1[16];
+#pragma unroll
+        for (int u = 0; u < 8; ++u) {
+          float4 v = make_float4(0.f, 0.f, 0.f, 0.f);
+          if (live && 32 * b + 4 * u < K) v = slot_ld4(box, row, 4 * u);
+          if (EPI == EPI_NODE) {
+            v.x *= xs; v.y *= xs; v.z *= xs; v.w *= xs;
+          }
+          split2(v.x, v.y, x0[2 * u], x1[2 * u]);
+          split2(v.z, v.w, x0[2 * u + 1], x1[2 * u + 1]);
+        }
+        tc::mbar_arrive(s.empty + sl);                         // box consumed (in registers)
+        tc::tmem_st16(lane_base + uint32_t(b * 16), x0);
+        tc::tmem_st16(lane_base + uint32_t(Kpad / 2 + b * 16), x1);
+      }
+      if (kh == 0) s.erow[(i & 3) * 128 + row] = er;
+      tc::tmem_st_wait();
+      tc::fence_before_sync();
+      tc::mbar_arrive(s.eready + (i & 3));
+      __syncwarp();
+      if (lane == 0) tc::mbar_arrive_cluster(s.afull, 0);
+    }
+    // the last tile's MMAs (and their commits to this CTA) must land before teardown
+    if (my > 0) tc::mbar_wait(s.afree, uint32_t(my - 1) & 1u);
+  } else {
+    // ---------------- epilogue: thread = (row, 64-channel quarter) ----------------
+    const int wi = warp - EPI0;
+    const int cq = wi >> 2;
+    const int qd = warp & 3;
+    const int row = qd * 32 + lane;
+    const uint32_t lane_base = tmem + (uint32_t(qd * 32) << 16);
+    float *wbuf = s.xbuf + wi * (16 * 20);
+    constexpr int DQ = PD / 4;
+    const int cb = cq * DQ;
+    for (int i = 0; i < my; ++i) {
+      const long r0 = row0_of(i);
+      const int nrows = int(max(0L, min(long(TM), a.R - r0)));
+      const bool live = row < nrows;
+      float aux = 0.f;
+      if (EPI == EPI_EDGE && live)
+        aux = __ldg(a.pin + __ldg(a.src + r0 + row)) + __ldg(a.qin + __ldg(a.dst + r0 + row));  // α
+      tc::mbar_wait(s.eready + (i & 3), uint32_t(i >> 2) & 1u);
+      const int er = s.erow[(i & 3) * 128 + row];
+      tc::mbar_wait(s.accfull, uint32_t(i) & 1u);
+      tc::fence_after_sync();
+      const float un = ldexpf(1.f, -(er + fexp));
+      const long grow = r0 + row;
+      const long wrow0 = r0 + qd * 32;
+      const int wrows = max(0, min(32, nrows - qd * 32));
+      const uint32_t acc = lane_base + 256u + uint32_t(cb);
+      if (EPI == EPI_GATE) {
+        float m = 0.f;
+        if (!noshift) {
+          m = -INFINITY;
+#pragma unroll
+          for (int c0 = 0; c0 < DQ; c0 += 16) {
+            uint32_t r[16];
+            tc::tmem_ld16(acc + c0, r);
+            tc::tmem_ld_wait();
+#pragma unroll
+            for (int u = 0; u < 16; ++u) m = fmaxf(m, __uint_as_float(r[u]) * un);
+          }
+          s.xch[cq * 128 + row] = m;
+          epi_bar_pair();
+          m = fmaxf(fmaxf(s.xch[row], s.xch[128 + row]), fmaxf(s.xch[256 + row], s.xch[384 + row]));
+        }
+        const float unL = un * LOG2E, mL = m * LOG2E;
+        float sum = 0.f;
+#pragma unroll
+        for (int c0 = 0; c0 < DQ; c0 += 16) {
+          uint32_t r[16];
+          tc::tmem_ld16(acc + c0, r);
+          tc::tmem_ld_wait();
+#pragma unroll
+          for (int u = 0; u < 16; ++u) sum += ex2(fmaf(__uint_as_float(r[u]), unL, -mL));
+        }
+        float *xs2 = s.xch + 512;
+        xs2[cq * 128 + row] = sum;
+        epi_bar_pair();
+        sum = ((xs2[row] + xs2[128 + row]) + xs2[256 + row]) + xs2[384 + row];   // fixed order
+        const float inv = fast_rcp(sum);
+#pragma unroll 1
+        for (int c0 = 0; c0 < DQ; c0 += 16) {
+          uint32_t r[16];
+          tc::tmem_ld16(acc + c0, r);
+          tc::tmem_ld_wait();
+          if (c0 + 16 >= DQ) {                                 // accumulator fully read
+            tc::fence_before_sync();
+            __syncwarp();
+            if (lane == 0) tc::mbar_arrive_cluster(s.accfree, 0);
+          }
+          float o[16];
+#pragma unroll
+          for (int u = 0; u < 16; ++u) o[u] = ex2(fmaf(__uint_as_float(r[u]), unL, -mL)) * inv;
+          warp_store_chunk<PD>(wbuf, a.out, wrow0, wrows, cb + c0, o, lane);
+        }
+      } else {
+        float pp = 0.f, qq = 0.f;
+#pragma unroll 1
+        for (int c0 = 0; c0 < DQ; c0 += 16) {
+          uint32_t r[16];
+          tc::tmem_ld16(acc + c0, r);
+          tc::tmem_ld_wait();
+          if (c0 + 16 >= DQ) {
+            tc::fence_before_sync();
+            __syncwarp();
+            if (lane == 0) tc::mbar_arrive_cluster(s.accfree, 0);
+          }
+          float o[16];
+#pragma unroll
+          for (int u = 0; u < 16; u += 4) {
+            if (EPI == EPI_NODE) {
+              const float4 as4 = *reinterpret_cast<const float4 *>(s.avec + cb + c0 + u);
+              const float4 ad4 = *reinterpret_cast<const float4 *>(s.avec + PD + cb + c0 + u);
+              const float asv[4] = {as4.x, as4.y, as4.z, as4.w};
+              const float adv[4] = {ad4.x, ad4.y, ad4.z, ad4.w};
+#pragma unroll
+              for (int t = 0; t < 4; ++t) {
+                o[u + t] = lrelu(__uint_as_float(r[u + t]) * un, a.slope);
+                pp = fmaf(o[u + t], asv[t], pp);
+                qq = fmaf(o[u + t], adv[t], qq);
+              }
+            } else {
+              const float cexp = -aux * un * LOG2E;
+#pragma unroll
+              for (int t = 0; t < 4; ++t) o[u + t] = fast_rcp(1.f + ex2(__uint_as_float(r[u + t]) * cexp));
+            }
+          }
+          warp_store_chunk<PD>(wbuf, a.out, wrow0, wrows, cb + c0, o, lane);
+        }
+        if (EPI == EPI_NODE) {
+          s.xch[cq * 128 + row] = pp;
+          s.xch[512 + cq * 128 + row] = qq;
+          epi_bar_pair();
+          if (cq == 0 && live) {
+            a.p[grow] = ((s.xch[row] + s.xch[128 + row]) + s.xch[256 + row]) + s.xch[384 + row];
+            a.q[grow] = ((s.xch[512 + row] + s.xch[640 + row]) + s.xch[768 + row]) + s.xch[896 + row];
+          }
+        }
+      }
+      epi_bar_pair();          // the exchange area is reused by the next tile
+    }
+  }
+  tc::fence_before_sync();
+  __syncthreads();
+  tc::cluster_sync();
+  tc::fence_after_sync();
+  if (warp == 1) tc::tmem_dealloc2<TMEM_COLS>(tmem);
+}
+
+// ---------------------------------------------------------------------------
 // Fused edge transform + channel-softmax gate of one ANEE layer (a3 + a4, P145/P149):
 //   e' = σ(α · W_e e_in), α = p[s] + q[t];   g = softmax_c(W_m e')
 // e' is written once (next layer's input, kept for the backward) and never re-read
@@ -1734,10 +2106,13 @@ int launch_wgrad_tc(const occu_ctx *ctx, const float *X, int A, const void *Y, i
   return 1;
 }
 
-constexpr size_t WIMG_MAX = size_t(2) * 128 * 128 * 2;   // [w0 | w1], Kpad <= 128, D <= 128
+// one image slot: [w0 | w1], Kpad <= 128 and D <= 128; at d = 256 Kpad, D <= 256
+static size_t wimg_slot_bytes(const occu_config &c) {
+  return c.d > 128 ? size_t(2) * 256 * 256 * 2 : size_t(2) * 128 * 128 * 2;
+}
 
 const uint8_t *tc_wimg(const occu_ctx *ctx, int kind, int layer) {
-  return ctx->wimg.as<uint8_t>() + size_t(layer * 6 + kind) * WIMG_MAX;
+  return ctx->wimg.as<uint8_t>() + size_t(layer * 6 + kind) * wimg_slot_bytes(ctx->cfg);
 }
 const int *tc_wfexp(const occu_ctx *ctx, int kind, int layer) {
   return ctx->wfexp.as<int>() + (layer * 6 + kind) * 2;     // [f, softmax no-shift flag]
@@ -1752,7 +2127,8 @@ int tc_prepare_weights(occu_ctx *ctx, cudaStream_t st) {
   // "layer" L + 1 + j for Graphormer layer j (kinds 0-5: W_q, W_k, W_v, W_o, FFN W1, W2)
   // + "layer" L + 1 + G + j: Graphormer layer j's transposed matrices (backward, gph_tslot)
   const size_t nslot = size_t(c.L + 1 + 2 * c.graphormer) * 6;
-  if (ctx->wimg.ensure(nslot * WIMG_MAX) != cudaSuccess ||
+  const int kmax = c.d > 128 ? 256 : 128;     // largest K an image slot holds
+  if (ctx->wimg.ensure(nslot * wimg_slot_bytes(c)) != cudaSuccess ||
       ctx->wfexp.ensure(nslot * 2 * sizeof(int)) != cudaSuccess ||
       ctx->wjobs.ensure(nslot * sizeof(WImageJob)) != cudaSuccess)
     return -int(cudaErrorMemoryAllocation);
@@ -1769,14 +2145,15 @@ int tc_prepare_weights(occu_ctx *ctx, cudaStream_t st) {
       j.fexp = const_cast<int *>(tc_wfexp(ctx, kind, i));
       jobs.push_back(j);
     };
-    if (L.d_in[i] <= 128) add(0, P + L.W_u[i], c.d, L.d_in[i], 0);
-    if (L.de_in[i] > 16 && L.de_in[i] <= 128) {
+    const bool fwd_only = c.d > 128;     // d = 256 runs inference only (no backward images)
+    if (L.d_in[i] <= kmax) add(0, P + L.W_u[i], c.d, L.d_in[i], 0);
+    if (L.de_in[i] > 16 && L.de_in[i] <= kmax) {
       add(1, P + L.W_e[i], c.d, L.de_in[i], 0);
-      add(4, P + L.W_e[i], c.d, c.d, 1);
+      if (!fwd_only) add(4, P + L.W_e[i], c.d, c.d, 1);
     }
     add(2, P + L.W_m[i], c.d, c.d, 0);
-    add(3, P + L.W_m[i], c.d, c.d, 1);
-    if (i > 0) add(5, P + L.W_u[i], c.d, c.d, 1);
+    if (!fwd_only) add(3, P + L.W_m[i], c.d, c.d, 1);
+    if (i > 0 && !fwd_only) add(5, P + L.W_u[i], c.d, c.d, 1);
   }
   if (L.dec) {      // NEXT-2 decoder: the pre-pooling FFN's two d x d matrices
     auto addd = [&](int kind, const float *W, int transW = 0) {
@@ -1821,7 +2198,7 @@ int tc_prepare_weights(occu_ctx *ctx, cudaStream_t st) {
 int gph_tslot(const occu_config &c, int j) { return c.L + 1 + c.graphormer + j; }
 
 bool tc_supported(const occu_config &c) {
-  return (c.d == 64 || c.d == 128) && c.F_n <= 128;
+  return ((c.d == 64 || c.d == 128) && c.F_n <= 128) || (c.d == 256 && c.F_n <= 256);
 }
 
 size_t tc_partial_floats(int E, int D) { return size_t(E / 32 + 2) * 2 * D; }
@@ -1841,6 +2218,74 @@ static int launch_rowgemm(const occu_ctx *ctx, const RowGemmArgs &ra, const char
   OCCU_PROF_END(ctx);
   TC_CHECK();
   return 1;
+}
+
+// d = 256: CTA-pair row-GEMM (rowgemm_pair_kernel), grid = 2 x clusters
+template <int EPI>
+static int launch_rowgemm_pair(const occu_ctx *ctx, const RowGemmArgs &ra, const char *name,
+                               cudaStream_t st) {
+  if (ra.R <= 0) return 0;
+  if (ra.K > 256) return -int(cudaErrorInvalidValue);
+  const size_t smem = pair_smem_bytes(ra.K);
+  set_smem(rowgemm_pair_kernel<EPI>, smem);
+  const int tiles = (ra.R + 2 * TM - 1) / (2 * TM);
+  const int clusters = std::max(1, std::min(tiles, ctx->num_sms / 2));
+  CUtensorMap tmap;
+  if (!encode_rows_map(&tmap, ra.A, ra.R, ra.K)) return -int(cudaErrorInvalidValue);
+  OCCU_PROF_BEGIN(ctx, name, st);
+  launch_pdl(ctx->pdl & 1, rowgemm_pair_kernel<EPI>, 2 * clusters, P_NTH, smem, st, tmap, ra);
+  OCCU_PROF_END(ctx);
+  TC_CHECK();
+  return 1;
+}
+
+// One ANEE layer at d = 256 (a2-a6), FP32: node transform, edge transform (CUDA cores for
+// F_e <= 16, else the pair GEMM), channel-softmax gate, then the CUDA-core aggregation.
+static int tc_forward_layer_pair(const occu_ctx *ctx, const DevCsr &csr, int layer,
+                                 const FwdLayerArgs &a, cudaStream_t st) {
+  constexpr int D = 256;
+  const float slope = ctx->cfg.slope;
+  int n = 0, r;
+  RowGemmArgs ra{};
+  ra.slope = slope;
+  ra.A = a.h_in; ra.K = a.K; ra.R = csr.N; ra.W = a.W_u; ra.out = a.hbar;
+  ra.wimg = tc_wimg(ctx, 0, layer); ra.wfexp = tc_wfexp(ctx, 0, layer);
+  ra.a_s = a.a_s; ra.a_d = a.a_d; ra.p = a.p; ra.q = a.q;
+  ra.rev = ctx->l2_order;
+  if ((r = launch_rowgemm_pair<EPI_NODE>(ctx, ra, "node_tc", st)) < 0) return r;
+  n += r;
+  if (csr.E > 0) {
+    if (a.Ke <= 16) {
+      const int grid = int(std::min<long>((long(csr.E) + 255) / 256, 8L * ctx->num_sms));
+      OCCU_PROF_BEGIN(ctx, "edge_small", st);
+      if (a.Ke <= 4)
+        launch_pdl(ctx->pdl & 4, edge_small_kernel<D, 4>, grid, 256, D * a.Ke * 4, st, a.e_in, a.Ke, a.W_e,
+                   a.p, a.q, csr.in_src, csr.in_dst, a.e_eid, csr.E, a.e_out, a.e0_out);
+      else
+        launch_pdl(ctx->pdl & 4, edge_small_kernel<D, 16>, grid, 256, D * a.Ke * 4, st, a.e_in, a.Ke, a.W_e,
+                   a.p, a.q, csr.in_src, csr.in_dst, a.e_eid, csr.E, a.e_out, a.e0_out);
+      OCCU_PROF_END(ctx);
+      TC_CHECK();
+      ++n;
+    } else {
+      RowGemmArgs re{};
+      re.slope = slope;
+      re.A = a.e_in; re.K = a.Ke; re.R = csr.E; re.W = a.W_e; re.out = a.e_out;
+      re.wimg = tc_wimg(ctx, 1, layer); re.wfexp = tc_wfexp(ctx, 1, layer);
+      re.pin = a.p; re.qin = a.q; re.src = csr.in_src; re.dst = csr.in_dst;
+      if ((r = launch_rowgemm_pair<EPI_EDGE>(ctx, re, "edge_tc", st)) < 0) return r;
+      n += r;
+    }
+    RowGemmArgs rg{};
+    rg.slope = slope;
+    rg.A = a.e_out; rg.K = D; rg.R = csr.E; rg.W = a.W_m; rg.out = a.g;
+    rg.wimg = tc_wimg(ctx, 2, layer); rg.wfexp = tc_wfexp(ctx, 2, layer);
+    rg.rev = ctx->l2_order;
+    if ((r = launch_rowgemm_pair<EPI_GATE>(ctx, rg, "gate_tc", st)) < 0) return r;
+    n += r;
+  }
+  if ((r = launch_gather_segsum(ctx, csr, a.g, a.hbar, a.h_out, a.rpart, st)) < 0) return r;
+  return n + r;
 }
 
 template <int D>
@@ -2097,6 +2542,9 @@ int launch_forward_layer_tc(const occu_ctx *ctx, const DevCsr &csr, int layer, c
   switch (ctx->cfg.d) {
     case 64: return tc_forward_layer_impl<64>(ctx, csr, layer, a, partial, st);
     case 128: return tc_forward_layer_impl<128>(ctx, csr, layer, a, partial, st);
+    case 256:
+      if (ctx->cfg.msg != OCCU_MSG_CHANNEL_SOFTMAX) return -int(cudaErrorInvalidValue);
+      return tc_forward_layer_pair(ctx, csr, layer, a, st);
     default: return -int(cudaErrorInvalidValue);
   }
 }

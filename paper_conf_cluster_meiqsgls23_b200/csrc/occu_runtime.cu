@@ -151,8 +151,12 @@ bool is_device_ptr(const void *p) {
 occu_status validate_cfg(const occu_config *c) {
   if (!c) return fail(nullptr, OCCU_EINVAL, "config is NULL");
   if (c->L < 1 || c->L > 16) return fail(nullptr, OCCU_EINVAL, "L must be in [1, 16]");
-  if (c->d != 64 && c->d != 128)
-    return fail(nullptr, OCCU_EINVAL, "this build supports d in {64, 128}");
+  if (c->d != 64 && c->d != 128 && c->d != 256)
+    return fail(nullptr, OCCU_EINVAL, "this build supports d in {64, 128, 256}");
+  if (c->d == 256 && (c->prec != OCCU_FP32 || c->msg != OCCU_MSG_CHANNEL_SOFTMAX ||
+                      c->readout != OCCU_READOUT_MEAN || c->graphormer != 0))
+    return fail(nullptr, OCCU_EINVAL,
+                "d = 256 (CTA-pair tensor-core path) supports OCCU_FP32, reading A, the mean readout and no Graphormer layers");
   if (c->F_n < 4 || c->F_n % 4 || c->F_n > 256 || c->F_e < 4 || c->F_e % 4 || c->F_e > 256)
     return fail(nullptr, OCCU_EINVAL, "F_n, F_e must be multiples of 4 in [4, 256]");
   if (c->d_h < 1 || c->d_h > 1024) return fail(nullptr, OCCU_EINVAL, "d_h must be in [1, 1024]");
@@ -427,6 +431,8 @@ occu_status check_train(occu_ctx *ctx, const occu_batch *batch, const float *tar
     return fail(ctx, OCCU_EINVAL, "training through the Graphormer layers / decoder readout runs in OCCU_FP32 on kernel path 0");
   if (ctx->cfg.msg == OCCU_MSG_NEIGHBOR_SOFTMAX && ctx->cfg.prec == OCCU_BF16)
     return fail(ctx, OCCU_EINVAL, "reading B in OCCU_BF16 is inference-only in this build");
+  if (ctx->cfg.d > 128)
+    return fail(ctx, OCCU_EINVAL, "d = 256 is inference-only in this build");
   return OCCU_OK;
 }
 

@@ -76,10 +76,13 @@ def capture(rep):
         except Exception:
             return None
     scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9}.get(rows[1][hdr.index("dram__bytes_read.sum")], 1)
+    tunit = rows[1][hdr.index("gpu__time_duration.sum")]
+    tscale = {"nsecond": 1e-3, "ns": 1e-3, "usecond": 1.0, "us": 1.0, "msecond": 1e3, "ms": 1e3,
+              "second": 1e6, "s": 1e6}[tunit]
     acc = collections.defaultdict(list)
     for r in rows[2:]:
         acc[kname(r[hdr.index("Kernel Name")])].append({
-            "time_us": g(r, "gpu__time_duration.sum") or 0,
+            "time_us": (g(r, "gpu__time_duration.sum") or 0) * tscale,
             "dram": ((g(r, "dram__bytes_read.sum") or 0) + (g(r, "dram__bytes_write.sum") or 0)) * scale,
             "dram_pct": g(r, "gpu__dram_throughput.avg.pct_of_peak_sustained_elapsed") or 0,
             "tensor": g(r, "sm__pipe_tensor_cycles_active.avg.pct_of_peak_sustained_elapsed") or 0,
@@ -100,7 +103,7 @@ def main():
     tag, lpath = sys.argv[1], sys.argv[2]
     os.makedirs(OUT, exist_ok=True)
     md = [f"# {tag}: ncu evidence (serialised, cold-cache replays; --clock-control none)\n"]
-    if os.path.exists(lpath):
+    if os.path.exists(lpath) and '"ID"' in open(lpath).read():
         md += [f"## launch list ({os.path.basename(lpath)})\n", launches(tag, lpath), ""]
     for spec in sys.argv[3:]:
         rep, title, tj = spec.split(":", 2)
