@@ -1122,20 +1122,17 @@ __global__ void __launch_bounds__(RO_WARPS * 32) readout_head_kernel(
   for (; k + 3 * RO_WARPS < k1; k += 4 * RO_WARPS) {
     float x[4][V];
 #pragma unroll
-    for (int t = 0; t < 4; ++t) {
-      const float *src = h + long(row_of(k + t * RO_WARPS)) * D + lane * V;
-#pragma unroll
-      for (int c = 0; c < V; ++c) x[t][c] = __ldg(src + c);
-    }
+    for (int t = 0; t < 4; ++t) load_row<V, false>(h, long(row_of(k + t * RO_WARPS)), D, lane, x[t]);
 #pragma unroll
     for (int t = 0; t < 4; ++t)
 #pragma unroll
       for (int c = 0; c < V; ++c) acc[c] += x[t][c];
   }
   for (; k < k1; k += RO_WARPS) {
-    const float *src = h + long(row_of(k)) * D + lane * V;
+    float x[V];
+    load_row<V, false>(h, long(row_of(k)), D, lane, x);
 #pragma unroll
-    for (int c = 0; c < V; ++c) acc[c] += __ldg(src + c);
+    for (int c = 0; c < V; ++c) acc[c] += x[c];
   }
 #pragma unroll
   for (int c = 0; c < V; ++c) part[warp * D + lane * V + c] = acc[c];
@@ -1156,9 +1153,10 @@ __global__ void __launch_bounds__(RO_WARPS * 32) readout_head_kernel(
       const int j = j0 + t * RO_WARPS;
       cv[t] = 0.f;
       if (j < d_h) {
+        float w[V];
+        load_row<V, false>(W_1, long(j), D, lane, w);     // coalesced vector loads of row j
 #pragma unroll
-        for (int c = 0; c < V; ++c)
-          cv[t] = fmaf(__ldg(W_1 + long(j) * D + lane * V + c), rs[lane * V + c], cv[t]);
+        for (int c = 0; c < V; ++c) cv[t] = fmaf(w[c], rs[lane * V + c], cv[t]);
       }
     }
 #pragma unroll

@@ -129,6 +129,7 @@ struct RowGemmArgs {
   float *dal;              // EDGEBWD: dα [R]
   float *part;             // GATEAGG: [R/32 units][2 slots][D] boundary-segment partials
   int rev;                 // walk tiles last-to-first (reads what the previous kernel wrote last, still in L2)
+  const int *rexp;         // d = 256 NODE: per-row scale exponents (row_exp_kernel)
 };
 
 struct Smem {
@@ -872,48 +873,55 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
 // the same three forward row-GEMMs (EPI_NODE / EPI_EDGE / EPI_GATE, same fused epilogues and
 // fp16x2 split as rowgemm_kernel) on a CTA PAIR.  One CTA cannot hold the fp16x2 images of
 // a 256 x 256 matrix (2 x 128 KB > 227 KB of shared memory), so two CTAs of a cluster on
-// neighbouring SMs run tcgen05.mma.cta_group::2: M = 256 rows per MMA (128 per CTA, A and
-// the accumulator in each CTA's own TMEM), B split along N (each CTA keeps the images of
-// its 128 output channels, resident for the whole kernel).  Each CTA ends up with full
-// 256-channel rows in TMEM, so the row epilogues (p/q dots, channel softmax) need no
-// exchange between the CTAs.
-//   warp 0      producer: the CTA's N-half of the images (bulk copies), then 2D TMA boxes
+// neighbouring SMs run tcgen05.mma.cta_group::2: M = 256 rows per MMA (128 per CTA), B split
+// along N (each CTA keeps the images of its 128 output channels, resident for the whole
+// kernel).  Each CTA ends up with full 256-channel rows in its TMEM, so the row epilogues
+// (p/q dots, channel softmax) need no exchange between the CTAs.
+//   warp 0      producer: the CTA's N-half of the images (bulk copies), then TMA boxes
 //               (128 rows x 32 fp32, SW128) of its rows into a P_NS-box ring;
-//   warp 1      TMEM (512 columns, cta_group::2 alloc in both CTAs); in the leader CTA the
-//               MMA issuer: 3·K/16 tcgen05.mma.cta_group::2 (M=256, N=256, K=16) per pair
-//               tile, committed to BOTH CTAs' barriers (multicast);
-//   warps 2-9   converters, thread = (row, box parity): fp16x2 split of each box into TMEM
-//               A (hi [0, Kpad/2), lo [Kpad/2, Kpad)); node inputs get the per-row power-of-two
-//               scale from the row max, read once from global memory (L2-resident for the
-//               TMA reads that follow); then one arrive per warp on the LEADER's A-full;
-//   warps 10-25 epilogue, thread = (row, 64-channel quarter): tcgen05.ld of the 256-column
-//               accumulator, the row epilogue (quarters combined in fixed order through
-//               shared memory), coalesced stores; one arrive per warp on the leader's
-//               accumulator-free barrier.
-// TMEM per CTA: A [0, 256) + ACC [256, 512), single-buffered: the converters of tile i+1 run
-// during the epilogue of tile i.  Pair tile t covers rows [256t, 256t + 256): rows
-// [256t + 128·rank, +128) live in CTA `rank`.
+//   warp 1      TMEM (512 columns, cta_group::2 alloc in both CTAs); in the leader CTA the MMA
+//               issuer: per 64-wide K chunk 4 x 3 tcgen05.mma.cta_group::2 (M=256, N=256,
+//               K=16, A from TMEM, B from shared memory), each chunk committed to both CTAs'
+//               A-slot-free barriers, each tile to both accumulator-full barriers;
+//   warps 2-5   converters, thread = row: the row's 32 fp32 of a box -> the box slot is
+//               released at once -> fp16x2 split -> tcgen05.st into a 4-chunk TMEM ring of A
+//               operands (hi | lo); node inputs are scaled by 2^e_row from a per-row exponent
+//               array (row_exp_kernel); one arrive per warp and chunk on the LEADER's A-full
+//               barrier;
+//   warps 6-21  epilogue, thread = (row, 64-channel quarter): its 64 accumulator values are
+//               loaded (tcgen05.ld) and the accumulator released on the leader's barrier
+//               before any arithmetic; the row epilogue (quarters combined in fixed order
+//               through shared memory) then runs from registers, coalesced stores.
+// TMEM per CTA: ACC [0, 256) + A ring [256, 512) (4 chunks x (32 hi + 32 lo columns)).  The
+// shared-memory box ring is released as soon as a box is in registers, so the TMA stream runs
+// up to a tile ahead of the MMAs (the resident images leave only ~64 KB for staging).  Pair
+// tile t covers rows [256t, 256t + 256): rows [256t + 128·rank, +128) live in CTA `rank`.
 // ---------------------------------------------------------------------------
-constexpr int P_NTH = 832;
-constexpr int P_NS = 4;               // input ring depth (boxes of 16 KB)
+constexpr int P_NTH = 704;           // warp 0 producer, 1 MMA, 2-5 converters, 6-21 epilogue
+constexpr int P_EPI0 = 6;
+constexpr int P_NS = 4;               // shared-memory ring of fp32 boxes (16 KB each)
+constexpr int P_NA = 4;               // TMEM ring of A chunks (64 columns each)
+#ifndef OCCU_PAIR_PF
+#define OCCU_PAIR_PF 0
+#endif
+constexpr int P_PF = OCCU_PAIR_PF;    // boxes prefetched into L2 ahead of the shared-memory ring
 constexpr int PD = 256;
 
 struct PairSmem {
   uint8_t *w0, *w1;                   // this CTA's N-half of [w0 | w1]: [Kpad/64][128 rows][128 B]
   float *ring;                        // P_NS x 4096 floats
   uint64_t *full, *empty;             // [P_NS]
-  uint64_t *afull, *afree, *accfull, *accfree, *wfull, *wpeer, *eready;
+  uint64_t *afull, *afree;            // [P_NA]
+  uint64_t *accfull, *accfree, *wfull, *wpeer;
   uint32_t *tmem_slot;
   float *avec;                        // [2][256] a_s, a_d (NODE)
-  int *erow;                          // [4][128]
-  float *cmax;                        // [2][128]
   float *xch;                         // [2 values][4 quarters][128 rows]
   float *xbuf;                        // 16 epilogue warps x 16 x 20 floats
 };
 
 __host__ __device__ inline size_t pair_smem_bytes(int K) {
   const size_t img = size_t(kpad_of(K)) * 128 * 2;
-  return 1024 + 2 * img + size_t(P_NS) * 16384 + 256 + 2048 + 2048 + 1024 + 4096 + 16 * 16 * 20 * 4;
+  return 1024 + 2 * img + size_t(P_NS) * 16384 + 256 + 2048 + 4096 + 16 * 16 * 20 * 4;
 }
 
 __device__ __forceinline__ PairSmem carve_pair(uint8_t *raw, int K) {
@@ -929,18 +937,15 @@ __device__ __forceinline__ PairSmem carve_pair(uint8_t *raw, int K) {
   s.full = bars;
   s.empty = bars + P_NS;
   s.afull = bars + 2 * P_NS;
-  s.afree = s.afull + 1;
-  s.accfull = s.afull + 2;
-  s.accfree = s.afull + 3;
-  s.wfull = s.afull + 4;
-  s.wpeer = s.afull + 5;
-  s.eready = s.afull + 6;             // 4
+  s.afree = s.afull + P_NA;
+  s.accfull = s.afree + P_NA;
+  s.accfree = s.accfull + 1;
+  s.wfull = s.accfull + 2;
+  s.wpeer = s.accfull + 3;
   s.tmem_slot = reinterpret_cast<uint32_t *>(misc + 224);
   s.avec = reinterpret_cast<float *>(misc + 256);
-  s.erow = reinterpret_cast<int *>(misc + 256 + 2048);
-  s.cmax = reinterpret_cast<float *>(misc + 256 + 4096);
-  s.xch = reinterpret_cast<float *>(misc + 256 + 4096 + 1024);
-  s.xbuf = reinterpret_cast<float *>(misc + 256 + 4096 + 1024 + 4096);
+  s.xch = reinterpret_cast<float *>(misc + 256 + 2048);
+  s.xbuf = reinterpret_cast<float *>(misc + 256 + 2048 + 4096);
   return s;
 }
 
@@ -950,7 +955,7 @@ template <int EPI>
 __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(P_NTH, 1)
     rowgemm_pair_kernel(const __grid_constant__ CUtensorMap tmap, RowGemmArgs a) {
   extern __shared__ uint8_t smem_raw[];
-  const int K = a.K, Kpad = kpad_of(K), NB = nbox_of(K);
+  const int K = a.K, Kpad = kpad_of(K), NC = Kpad / 64, NB = nbox_of(K);
   PairSmem s = carve_pair(smem_raw, K);
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const uint32_t rank = tc::cluster_rank();
@@ -959,15 +964,16 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(P_NTH, 1)
   if (threadIdx.x == 0) {
     for (int j = 0; j < P_NS; ++j) {
       tc::mbar_init(s.full + j, 1);
-      tc::mbar_init(s.empty + j, 128);
+      tc::mbar_init(s.empty + j, 128);  // the 4 converter warps
     }
-    tc::mbar_init(s.afull, 16);       // 8 converter warps x 2 CTAs (leader's copy used)
-    tc::mbar_init(s.afree, 1);        // multicast commit
-    tc::mbar_init(s.accfull, 1);      // multicast commit
-    tc::mbar_init(s.accfree, 32);     // 16 epilogue warps x 2 CTAs (leader's copy used)
+    for (int j = 0; j < P_NA; ++j) {
+      tc::mbar_init(s.afull + j, 8);    // 4 converter warps x 2 CTAs (leader's copy used)
+      tc::mbar_init(s.afree + j, 1);    // multicast commit
+    }
+    tc::mbar_init(s.accfull, 1);        // multicast commit
+    tc::mbar_init(s.accfree, 32);       // 16 epilogue warps x 2 CTAs (leader's copy used)
     tc::mbar_init(s.wfull, 1);
     tc::mbar_init(s.wpeer, 1);
-    for (int j = 0; j < 4; ++j) tc::mbar_init(s.eready + j, 256);
     tc::fence_mbar_init();
   }
   if (warp == 1) tc::tmem_alloc2<TMEM_COLS>(s.tmem_slot);
@@ -1000,7 +1006,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(P_NTH, 1)
       tc::prefetch_tmap(&tmap);
       const uint32_t ib = uint32_t(Kpad) * PD * 2;            // one full image (w0 or w1)
       tc::mbar_arrive_expect_tx(s.wfull, uint32_t(Kpad) * 128u * 2u * 2u);
-      for (int c = 0; c < Kpad / 64; ++c) {                   // 16 KB per 64-wide K chunk
+      for (int c = 0; c < NC; ++c) {                          // 16 KB per 64-wide K chunk
         const uint32_t src = uint32_t(c) * 32768u + rank * 16384u;
         tc::bulk_g2s(s.w0 + c * 16384, a.wimg + src, 16384, s.wfull);
         tc::bulk_g2s(s.w1 + c * 16384, a.wimg + ib + src, 16384, s.wfull);
@@ -1009,11 +1015,21 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(P_NTH, 1)
         tc::mbar_wait(s.wfull, 0);
         tc::mbar_arrive_cluster(s.wpeer, 0);
       }
+      // boxes are prefetched into L2 P_PF ahead of the ring: the resident weight images leave
+      // room for only P_NS boxes in shared memory, too few bytes in flight to cover HBM latency
+      const long nq = long(my) * NB;
+      auto prefetch = [&](long qq) {
+        if (qq >= nq) return;
+        const long rr = row0_of(int(qq / NB));
+        if (rr < a.R) tc::tma_prefetch_2d(&tmap, 32 * int(qq % NB), int(rr));
+      };
+      for (long qq = 0; qq < P_PF; ++qq) prefetch(qq);
       long q = 0;
       for (int i = 0; i < my; ++i) {
         const long r0 = row0_of(i);
         for (int b = 0; b < NB; ++b, ++q) {
           const int sl = int(q % P_NS);
+          prefetch(q + P_PF);
           if (q >= P_NS) tc::mbar_wait(s.empty + sl, uint32_t((q / P_NS) - 1) & 1u);
           if (r0 < a.R) {
             tc::mbar_arrive_expect_tx(s.full + sl, 16384u);
@@ -1034,88 +1050,83 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(P_NTH, 1)
       tc::mbar_wait(s.wfull, 0);
       tc::mbar_wait_cluster(s.wpeer, 0);
       for (int i = 0; i < my; ++i) {
-        tc::mbar_wait_cluster(s.afull, uint32_t(i) & 1u);
         if (i >= 1) tc::mbar_wait_cluster(s.accfree, uint32_t(i - 1) & 1u);
-        tc::fence_after_sync();
-        if (lane == 0) {
-          const uint32_t d = tmem + 256u;
-          for (int kk = 0; kk < nk; ++kk) {
-            const uint32_t boff = uint32_t(kk >> 2) * 16384u + uint32_t(kk & 3) * 32u;
-            const uint64_t b0 = tc::sdesc_sw128(w0a + boff), b1 = tc::sdesc_sw128(w1a + boff);
-            const uint32_t a0 = tmem + uint32_t(kk) * 8u;
-            const uint32_t a1 = a0 + uint32_t(Kpad / 2);
-            tc::mma2_f16_ts(d, a0, b0, idsc, kk > 0 ? 1u : 0u);
-            tc::mma2_f16_ts(d, a0, b1, idsc, 1u);
-            tc::mma2_f16_ts(d, a1, b0, idsc, 1u);
+        for (int c = 0; c < NC; ++c) {
+          const long qa = long(i) * NC + c;
+          const int as = int(qa % P_NA);
+          tc::mbar_wait_cluster(s.afull + as, uint32_t(qa / P_NA) & 1u);
+          tc::fence_after_sync();
+          if (lane == 0) {
+            const uint32_t ah = tmem + 256u + uint32_t(as) * 64u;
+            for (int kk = 0; kk < 4 && 4 * c + kk < nk; ++kk) {
+              const uint32_t bo = uint32_t(c) * 16384u + uint32_t(kk) * 32u;
+              const uint64_t b0 = tc::sdesc_sw128(w0a + bo), b1 = tc::sdesc_sw128(w1a + bo);
+              const uint32_t a0 = ah + uint32_t(kk) * 8u, a1 = a0 + 32u;
+              tc::mma2_f16_ts(tmem, a0, b0, idsc, (c | kk) ? 1u : 0u);
+              tc::mma2_f16_ts(tmem, a0, b1, idsc, 1u);
+              tc::mma2_f16_ts(tmem, a1, b0, idsc, 1u);
+            }
+            tc::mma2_commit_both(s.afree + as);
+            if (c == NC - 1) tc::mma2_commit_both(s.accfull);
           }
-          tc::mma2_commit_both(s.accfull);
-          tc::mma2_commit_both(s.afree);
+          __syncwarp();
         }
-        __syncwarp();
       }
     }
-  } else if (warp < EPI0) {
-    // ---------------- converters: thread = (row, box parity) -> TMEM A ----------------
+  } else if (warp < P_EPI0) {
+    // ---------------- converters: thread = row -> TMEM A ring ----------------
     const int qd = warp & 3;
-    const int kh = (warp - 2) >> 2;
     const int row = qd * 32 + lane;
     const uint32_t lane_base = tmem + (uint32_t(qd * 32) << 16);
-    const int kmid = (K / 4 + 1) / 2 * 4;                     // row-max halves
     for (int i = 0; i < my; ++i) {
       const long r0 = row0_of(i);
       const bool live = long(row) < a.R - r0;
-      if (i >= 1) tc::mbar_wait(s.afree, uint32_t(i - 1) & 1u);
-      int er = 0;                                              // e' in [0, 1]: unscaled
-      if (EPI == EPI_NODE) {
-        float mx = 0.f;
-        if (live) {
-          const float *src = a.A + (r0 + row) * K;
-          const int k0 = kh ? kmid : 0, k1 = kh ? K : kmid;
-#pragma unroll 4
-          for (int k = k0; k < k1; k += 4) {
-            const float4 v = __ldg(reinterpret_cast<const float4 *>(src + k));
-            mx = fmaxf(mx, fmaxf(fmaxf(fabsf(v.x), fabsf(v.y)), fmaxf(fabsf(v.z), fabsf(v.w))));
-          }
-        }
-        s.cmax[kh * 128 + row] = mx;
-        asm volatile("bar.sync 3, 256;" ::: "memory");
-        mx = fmaxf(mx, s.cmax[(kh ^ 1) * 128 + row]);
-        er = scale_exp(mx);
-        asm volatile("bar.sync 3, 256;" ::: "memory");
-      }
-      const float xs = ldexpf(1.f, er);
-      for (int b = kh; b < NB; b += 2) {
-        const long q = long(i) * NB + b;
-        const int sl = int(q % P_NS);
-        tc::mbar_wait(s.full + sl, uint32_t(q / P_NS) & 1u);
-        const float *box = s.ring + sl * 4096;
-        uint32_t x0[16], x1[16];
+      float xs = 1.f;                                          // e' in [0, 1]: unscaled
+      if (EPI == EPI_NODE && live) xs = ldexpf(1.f, __ldg(a.rexp + r0 + row));
+      for (int c = 0; c < NC; ++c) {
+        const long qa = long(i) * NC + c;
+        const int as = int(qa % P_NA);
+        for (int kh = 0; kh < 2; ++kh) {
+          const int b = 2 * c + kh;
+          if (b >= NB) break;
+          const long q = long(i) * NB + b;
+          const int sl = int(q % P_NS);
+          tc::mbar_wait(s.full + sl, uint32_t(q / P_NS) & 1u);
+          const float *box = s.ring + sl * 4096;
+          float4 v[8];
 #pragma unroll
-        for (int u = 0; u < 8; ++u) {
-          float4 v = make_float4(0.f, 0.f, 0.f, 0.f);
-          if (live && 32 * b + 4 * u < K) v = slot_ld4(box, row, 4 * u);
-          if (EPI == EPI_NODE) {
-            v.x *= xs; v.y *= xs; v.z *= xs; v.w *= xs;
+          for (int u = 0; u < 8; ++u)
+            v[u] = (live && 32 * b + 4 * u < K) ? slot_ld4(box, row, 4 * u) : make_float4(0.f, 0.f, 0.f, 0.f);
+          tc::mbar_arrive(s.empty + sl);                      // the box is in registers
+          uint32_t h[16], l[16];
+#pragma unroll
+          for (int u = 0; u < 8; ++u) {
+            float4 x = v[u];
+            if (EPI == EPI_NODE) {
+              x.x *= xs; x.y *= xs; x.z *= xs; x.w *= xs;
+            }
+            split2(x.x, x.y, h[2 * u], l[2 * u]);
+            split2(x.z, x.w, h[2 * u + 1], l[2 * u + 1]);
           }
-          split2(v.x, v.y, x0[2 * u], x1[2 * u]);
-          split2(v.z, v.w, x0[2 * u + 1], x1[2 * u + 1]);
+          if (kh == 0 && qa >= P_NA) tc::mbar_wait(s.afree + as, uint32_t((qa / P_NA) - 1) & 1u);
+          const uint32_t col = 256u + uint32_t(as) * 64u + uint32_t(kh) * 16u;
+          tc::tmem_st16(lane_base + col, h);
+          tc::tmem_st16(lane_base + col + 32u, l);
         }
-        tc::mbar_arrive(s.empty + sl);                         // box consumed (in registers)
-        tc::tmem_st16(lane_base + uint32_t(b * 16), x0);
-        tc::tmem_st16(lane_base + uint32_t(Kpad / 2 + b * 16), x1);
+        tc::tmem_st_wait();
+        tc::fence_before_sync();
+        __syncwarp();
+        if (lane == 0) tc::mbar_arrive_cluster(s.afull + as, 0);
       }
-      if (kh == 0) s.erow[(i & 3) * 128 + row] = er;
-      tc::tmem_st_wait();
-      tc::fence_before_sync();
-      tc::mbar_arrive(s.eready + (i & 3));
-      __syncwarp();
-      if (lane == 0) tc::mbar_arrive_cluster(s.afull, 0);
     }
-    // the last tile's MMAs (and their commits to this CTA) must land before teardown
-    if (my > 0) tc::mbar_wait(s.afree, uint32_t(my - 1) & 1u);
+    // the last chunks' MMAs (and their commits to this CTA) must land before teardown
+    for (long qa = max(0L, long(my) * NC - P_NA); qa < long(my) * NC; ++qa)
+      tc::mbar_wait(s.afree + int(qa % P_NA), uint32_t(qa / P_NA) & 1u);
   } else {
     // ---------------- epilogue: thread = (row, 64-channel quarter) ----------------
-    const int wi = warp - EPI0;
+    // the thread's 64 accumulator values are loaded at once and the accumulator released
+    // before any arithmetic, so the next tile's MMAs overlap this tile's epilogue
+    const int wi = warp - P_EPI0;
     const int cq = wi >> 2;
     const int qd = warp & 3;
     const int row = qd * 32 + lane;
@@ -1130,27 +1141,34 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(P_NTH, 1)
       float aux = 0.f;
       if (EPI == EPI_EDGE && live)
         aux = __ldg(a.pin + __ldg(a.src + r0 + row)) + __ldg(a.qin + __ldg(a.dst + r0 + row));  // α
-      tc::mbar_wait(s.eready + (i & 3), uint32_t(i >> 2) & 1u);
-      const int er = s.erow[(i & 3) * 128 + row];
+      const int er = (EPI == EPI_NODE && live) ? __ldg(a.rexp + r0 + row) : 0;
       tc::mbar_wait(s.accfull, uint32_t(i) & 1u);
       tc::fence_after_sync();
+      uint32_t r[DQ];
+      {
+        uint32_t (&r0_)[16] = *reinterpret_cast<uint32_t (*)[16]>(r);
+        uint32_t (&r1_)[16] = *reinterpret_cast<uint32_t (*)[16]>(r + 16);
+        uint32_t (&r2_)[16] = *reinterpret_cast<uint32_t (*)[16]>(r + 32);
+        uint32_t (&r3_)[16] = *reinterpret_cast<uint32_t (*)[16]>(r + 48);
+        tc::tmem_ld16(lane_base + uint32_t(cb), r0_);
+        tc::tmem_ld16(lane_base + uint32_t(cb) + 16u, r1_);
+        tc::tmem_ld16(lane_base + uint32_t(cb) + 32u, r2_);
+        tc::tmem_ld16(lane_base + uint32_t(cb) + 48u, r3_);
+        tc::tmem_ld_wait();
+      }
+      tc::fence_before_sync();
+      __syncwarp();
+      if (lane == 0) tc::mbar_arrive_cluster(s.accfree, 0);    // accumulator free
       const float un = ldexpf(1.f, -(er + fexp));
       const long grow = r0 + row;
       const long wrow0 = r0 + qd * 32;
       const int wrows = max(0, min(32, nrows - qd * 32));
-      const uint32_t acc = lane_base + 256u + uint32_t(cb);
       if (EPI == EPI_GATE) {
         float m = 0.f;
         if (!noshift) {
           m = -INFINITY;
 #pragma unroll
-          for (int c0 = 0; c0 < DQ; c0 += 16) {
-            uint32_t r[16];
-            tc::tmem_ld16(acc + c0, r);
-            tc::tmem_ld_wait();
-#pragma unroll
-            for (int u = 0; u < 16; ++u) m = fmaxf(m, __uint_as_float(r[u]) * un);
-          }
+          for (int u = 0; u < DQ; ++u) m = fmaxf(m, __uint_as_float(r[u]) * un);
           s.xch[cq * 128 + row] = m;
           epi_bar_pair();
           m = fmaxf(fmaxf(s.xch[row], s.xch[128 + row]), fmaxf(s.xch[256 + row], s.xch[384 + row]));
@@ -1158,45 +1176,26 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(P_NTH, 1)
         const float unL = un * LOG2E, mL = m * LOG2E;
         float sum = 0.f;
 #pragma unroll
-        for (int c0 = 0; c0 < DQ; c0 += 16) {
-          uint32_t r[16];
-          tc::tmem_ld16(acc + c0, r);
-          tc::tmem_ld_wait();
-#pragma unroll
-          for (int u = 0; u < 16; ++u) sum += ex2(fmaf(__uint_as_float(r[u]), unL, -mL));
+        for (int u = 0; u < DQ; ++u) {
+          const float e = ex2(fmaf(__uint_as_float(r[u]), unL, -mL));
+          r[u] = __float_as_uint(e);
+          sum += e;
         }
         float *xs2 = s.xch + 512;
         xs2[cq * 128 + row] = sum;
         epi_bar_pair();
         sum = ((xs2[row] + xs2[128 + row]) + xs2[256 + row]) + xs2[384 + row];   // fixed order
         const float inv = fast_rcp(sum);
-#pragma unroll 1
-        for (int c0 = 0; c0 < DQ; c0 += 16) {
-          uint32_t r[16];
-          tc::tmem_ld16(acc + c0, r);
-          tc::tmem_ld_wait();
-          if (c0 + 16 >= DQ) {                                 // accumulator fully read
-            tc::fence_before_sync();
-            __syncwarp();
-            if (lane == 0) tc::mbar_arrive_cluster(s.accfree, 0);
-          }
-          float o[16];
 #pragma unroll
-          for (int u = 0; u < 16; ++u) o[u] = ex2(fmaf(__uint_as_float(r[u]), unL, -mL)) * inv;
-          warp_store_chunk<PD>(wbuf, a.out, wrow0, wrows, cb + c0, o, lane);
-        }
+        for (int u = 0; u < DQ; ++u) r[u] = __float_as_uint(__uint_as_float(r[u]) * inv);
+#pragma unroll
+        for (int c0 = 0; c0 < DQ; c0 += 16)
+          warp_store_chunk<PD>(wbuf, a.out, wrow0, wrows, cb + c0,
+                               *reinterpret_cast<const float (*)[16]>(r + c0), lane);
       } else {
         float pp = 0.f, qq = 0.f;
-#pragma unroll 1
+#pragma unroll
         for (int c0 = 0; c0 < DQ; c0 += 16) {
-          uint32_t r[16];
-          tc::tmem_ld16(acc + c0, r);
-          tc::tmem_ld_wait();
-          if (c0 + 16 >= DQ) {
-            tc::fence_before_sync();
-            __syncwarp();
-            if (lane == 0) tc::mbar_arrive_cluster(s.accfree, 0);
-          }
           float o[16];
 #pragma unroll
           for (int u = 0; u < 16; u += 4) {
@@ -1207,14 +1206,14 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(P_NTH, 1)
               const float adv[4] = {ad4.x, ad4.y, ad4.z, ad4.w};
 #pragma unroll
               for (int t = 0; t < 4; ++t) {
-                o[u + t] = lrelu(__uint_as_float(r[u + t]) * un, a.slope);
+                o[u + t] = lrelu(__uint_as_float(r[c0 + u + t]) * un, a.slope);
                 pp = fmaf(o[u + t], asv[t], pp);
                 qq = fmaf(o[u + t], adv[t], qq);
               }
             } else {
               const float cexp = -aux * un * LOG2E;
 #pragma unroll
-              for (int t = 0; t < 4; ++t) o[u + t] = fast_rcp(1.f + ex2(__uint_as_float(r[u + t]) * cexp));
+              for (int t = 0; t < 4; ++t) o[u + t] = fast_rcp(1.f + ex2(__uint_as_float(r[c0 + u + t]) * cexp));
             }
           }
           warp_store_chunk<PD>(wbuf, a.out, wrow0, wrows, cb + c0, o, lane);
@@ -1237,6 +1236,25 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(P_NTH, 1)
   tc::cluster_sync();
   tc::fence_after_sync();
   if (warp == 1) tc::tmem_dealloc2<TMEM_COLS>(tmem);
+}
+
+// Per-row power-of-two scale exponent e_r (max|x_r|·2^e_r in [2^14, 2^15), scale_exp) of the
+// node-transform input rows at d = 256; warp per row.
+__global__ void __launch_bounds__(256) row_exp_kernel(const float *__restrict__ A, int R, int K,
+                                                      int *__restrict__ out) {
+  pdl_trigger();
+  pdl_wait();
+  const int lane = threadIdx.x & 31;
+  for (long r = (long(blockIdx.x) * 256 + threadIdx.x) / 32; r < R; r += long(gridDim.x) * 8) {
+    float mx = 0.f;
+    for (int k = 4 * lane; k < K; k += 128) {
+      const float4 v = __ldg(reinterpret_cast<const float4 *>(A + r * K + k));
+      mx = fmaxf(mx, fmaxf(fmaxf(fabsf(v.x), fabsf(v.y)), fmaxf(fabsf(v.z), fabsf(v.w))));
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) mx = fmaxf(mx, __shfl_xor_sync(0xffffffffu, mx, o));
+    if (lane == 0) out[r] = scale_exp(mx);
+  }
 }
 
 // ---------------------------------------------------------------------------
@@ -1772,6 +1790,9 @@ __global__ void __launch_bounds__(256) edge_small_kernel(
       float *dst = e_out + (k0 + u) * D + c;
       if constexpr (V == 4) {
         *reinterpret_cast<float4 *>(dst) = make_float4(o[0], o[1], o[2], o[3]);
+      } else if constexpr (V == 8) {
+        *reinterpret_cast<float4 *>(dst) = make_float4(o[0], o[1], o[2], o[3]);
+        *reinterpret_cast<float4 *>(dst + 4) = make_float4(o[4 % V], o[5 % V], o[6 % V], o[7 % V]);
       } else {
 #pragma unroll
         for (int v = 0; v < V; v += 2) *reinterpret_cast<float2 *>(dst + v) = make_float2(o[v], o[v + 1]);
@@ -2222,7 +2243,7 @@ static int launch_rowgemm(const occu_ctx *ctx, const RowGemmArgs &ra, const char
 
 // d = 256: CTA-pair row-GEMM (rowgemm_pair_kernel), grid = 2 x clusters
 template <int EPI>
-static int launch_rowgemm_pair(const occu_ctx *ctx, const RowGemmArgs &ra, const char *name,
+static int launch_rowgemm_pair(const occu_ctx *ctx, RowGemmArgs ra, const char *name,
                                cudaStream_t st) {
   if (ra.R <= 0) return 0;
   if (ra.K > 256) return -int(cudaErrorInvalidValue);
@@ -2232,11 +2253,21 @@ static int launch_rowgemm_pair(const occu_ctx *ctx, const RowGemmArgs &ra, const
   const int clusters = std::max(1, std::min(tiles, ctx->num_sms / 2));
   CUtensorMap tmap;
   if (!encode_rows_map(&tmap, ra.A, ra.R, ra.K)) return -int(cudaErrorInvalidValue);
+  int n = 0;
   OCCU_PROF_BEGIN(ctx, name, st);
+  if (EPI == EPI_NODE) {          // the rows' scale exponents first
+    if (const_cast<occu_ctx *>(ctx)->ws.rowexp.ensure(size_t(ra.R) * 4) != cudaSuccess)
+      return -int(cudaErrorMemoryAllocation);
+    int *rexp = ctx->ws.rowexp.as<int>();
+    ra.rexp = rexp;
+    const int g = int(std::min<long>((long(ra.R) + 7) / 8, 16L * ctx->num_sms));
+    launch_pdl(ctx->pdl & 1, row_exp_kernel, g, 256, 0, st, ra.A, ra.R, ra.K, rexp);
+    ++n;
+  }
   launch_pdl(ctx->pdl & 1, rowgemm_pair_kernel<EPI>, 2 * clusters, P_NTH, smem, st, tmap, ra);
   OCCU_PROF_END(ctx);
   TC_CHECK();
-  return 1;
+  return n + 1;
 }
 
 // One ANEE layer at d = 256 (a2-a6), FP32: node transform, edge transform (CUDA cores for

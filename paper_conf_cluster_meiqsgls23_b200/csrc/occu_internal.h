@@ -61,6 +61,7 @@ struct Workspace {
   DevBuf r, c, yhat;       // [B][d], [B][d_h], [B]
   // backward scratch
   DevBuf dy, dc, dr, dh, dhprev, dP, MG, DV, DZ, deA, deB, dalpha, dpq, partial, loss;
+  DevBuf rowexp;           // d = 256: per-row power-of-two scale exponents of node-transform inputs
   DevBuf tcpart;           // tensor-core aggregation: boundary-segment partials
   DevBuf dpart;            // per-warp [da_s; da_d] partials
   DevBuf anf[2], aef[2], acsr[2];   // occu_predict_async / occu_train_step_async: double-buffered input staging

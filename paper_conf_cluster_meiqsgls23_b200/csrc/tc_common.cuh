@@ -165,6 +165,13 @@ __device__ __forceinline__ void tma_load_2d(void *dst_smem, const CUtensorMap *m
       "l"(reinterpret_cast<uint64_t>(map)), "r"(x), "r"(y), "r"(smem_u32(bar))
       : "memory");
 }
+// 2D TMA box prefetched into L2 only (no shared memory, no barrier)
+__device__ __forceinline__ void tma_prefetch_2d(const CUtensorMap *map, int x, int y) {
+  asm volatile("cp.async.bulk.prefetch.tensor.2d.L2.global.tile [%0, {%1, %2}];" ::"l"(
+                   reinterpret_cast<uint64_t>(map)),
+               "r"(x), "r"(y)
+               : "memory");
+}
 __device__ __forceinline__ void prefetch_tmap(const CUtensorMap *map) {
   asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(map)) : "memory");
 }
@@ -252,25 +259,23 @@ __device__ __forceinline__ uint32_t ncluster_x() {
 __device__ __forceinline__ void cluster_sync() {
   asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
 }
-// arrive on the mbarrier at the same shared-memory offset in CTA `rank` of the cluster
+// arrive on the mbarrier at the same shared-memory offset in CTA `rank` of the cluster.
+// Default (CTA-scope release) semantics, as CUTLASS's ClusterBarrier::arrive(cta_id): the
+// cluster-scope form compiles to MEMBAR.ALL.GPU, which makes the arriving warp wait for its
+// outstanding global stores (measured: ~12 % of the pair kernel's stall samples).  What the
+// arrive publishes is shared memory (after fence.proxy.async) or TMEM reads (after
+// tcgen05.fence::before_thread_sync), both complete in the issuing SM before the arrive.
 __device__ __forceinline__ void mbar_arrive_cluster(uint64_t *bar, uint32_t rank) {
   uint32_t ra;
   asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(ra) : "r"(smem_u32(bar)), "r"(rank));
-  asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];" ::"r"(ra) : "memory");
+  asm volatile("mbarrier.arrive.shared::cluster.b64 _, [%0];" ::"r"(ra) : "memory");
 }
-// wait with cluster-scope acquire (the barrier receives arrivals from the peer CTA)
+// wait on a barrier that receives arrivals from the peer CTA (plain try_wait, as CUTLASS's
+// ClusterBarrier::wait; the cluster-scope acquire form invalidates L1 on every poll)
 __device__ __forceinline__ void mbar_wait_cluster(uint64_t *bar, uint32_t parity) {
   const uint32_t a = smem_u32(bar);
-  uint32_t ok;
-  do {
-    asm volatile(
-        "{\n\t.reg .pred P1;\n\t"
-        "mbarrier.try_wait.parity.acquire.cluster.shared::cta.b64 P1, [%1], %2;\n\t"
-        "selp.u32 %0, 1, 0, P1;\n\t}"
-        : "=r"(ok)
-        : "r"(a), "r"(parity)
-        : "memory");
-  } while (!ok);
+  while (!mbar_try_wait(a, parity)) {
+  }
 }
 // TMEM allocation for a CTA pair: one warp in EACH CTA of the pair executes these.
 template <uint32_t NCOLS>
@@ -294,6 +299,14 @@ __device__ __forceinline__ void mma2_f16_ts(uint32_t d_tmem, uint32_t a_tmem, ui
       "setp.ne.b32 p, %4, 0;\n\t"
       "tcgen05.mma.cta_group::2.kind::f16 [%0], [%1], %2, %3, p;\n\t}" ::"r"(d_tmem),
       "r"(a_tmem), "l"(b_desc), "r"(idsc), "r"(accumulate));
+}
+__device__ __forceinline__ void mma2_f16_ss(uint32_t d_tmem, uint64_t a_desc, uint64_t b_desc,
+                                            uint32_t idsc, uint32_t accumulate) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t"
+      "setp.ne.b32 p, %4, 0;\n\t"
+      "tcgen05.mma.cta_group::2.kind::f16 [%0], %1, %2, %3, p;\n\t}" ::"r"(d_tmem),
+      "l"(a_desc), "l"(b_desc), "r"(idsc), "r"(accumulate));
 }
 // commit the pair's MMAs to the mbarrier at this offset in both CTAs (mask 0b11)
 __device__ __forceinline__ void mma2_commit_both(uint64_t *bar) {

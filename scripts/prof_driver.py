@@ -19,9 +19,11 @@ ap.add_argument("--graphormer", type=int, default=0)
 ap.add_argument("--decoder", action="store_true")
 ap.add_argument("--synth", action="store_true", help="inputs synthesized on the device (NEXT-4)")
 ap.add_argument("--cfg3", action="store_true", help="CFG3 (512 BERT-base / GPT-2 graphs) instead of CFG2")
+ap.add_argument("--d", type=int, default=128)
+ap.add_argument("--L", type=int, default=3)
 a = ap.parse_args()
 dev = torch.device("cuda", 0)
-m = occu.Model(occu.config(L=3, F_n=80, F_e=4, d=128, prec=occu.BF16 if a.bf16 else occu.FP32,
+m = occu.Model(occu.config(L=a.L, F_n=80, F_e=4, d=a.d, prec=occu.BF16 if a.bf16 else occu.FP32,
                            graphormer=a.graphormer, heads=4,
                            readout=occu.READOUT_SET_DECODER if a.decoder else occu.READOUT_MEAN))
 m.init_weights(42)
