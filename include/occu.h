@@ -59,21 +59,27 @@ typedef enum { OCCU_FP32 = 0, OCCU_BF16 = 1 } occu_precision;
 
 typedef enum { OCCU_READOUT_MEAN = 0, OCCU_READOUT_SET_DECODER = 1 } occu_readout;
 
-/* Model configuration.  L ANEE rounds of width d (64 or 128 in this build); raw feature
+/* Model configuration.  L ANEE rounds of width d (64, 128 or 256); d = 256 is the paper's
+ * hidden width (P273) and runs on the CTA-pair tensor-core path: OCCU_FP32,
+ * msg = OCCU_MSG_CHANNEL_SOFTMAX, readout MEAN, graphormer = 0, F_n <= 256, inference only
+ * (occu_train_step / occu_grads return OCCU_EINVAL; any other d, or d = 256 with another
+ * mode, fails occu_create with OCCU_EINVAL).  Raw feature
  * widths F_n (node, Table I) and F_e (edge); head hidden width d_h; LeakyReLU slope (R7,
  * 0.01); F_n, F_e multiples of 4.  msg = OCCU_MSG_NEIGHBOR_SOFTMAX (reading B, NEXT-1):
  * kernel path 0; OCCU_FP32 forward + training, OCCU_BF16 forward (training with OCCU_BF16
  * returns OCCU_EINVAL: DESIGN.md R40).  readout: OCCU_READOUT_MEAN (a7, the north_star's segmented
  * mean; default when the trailing fields are zero) or OCCU_READOUT_SET_DECODER (P159-P205,
  * NEXT-2: Decoder(H) = FFN(SAB(PMA_k(H))) per graph, k seeds, `heads` attention heads, the
- * head reading the flattened k·d output; kernel path 0, inference only: training returns
- * OCCU_EINVAL; with OCCU_BF16 the decoder runs in FP32 on the BF16-stored h_L, R41);
+ * head reading the flattened k·d output; kernel path 0; training in OCCU_FP32 (R46;
+ * with OCCU_BF16 training returns OCCU_EINVAL and inference runs the decoder in FP32 on the
+ * BF16-stored h_L, R41);
  * k in [1, 8], heads in {1, 2, 4, 8}, k·heads <= 16.
  * graphormer: number of Graphormer layers (P153-P157, NEXT-3; R35-R37) between the
  * last ANEE round and the readout, h̄ = MHA(LN(h)) + h, h' = FFN(LN(h̄)) + h̄ with
  * self-attention over each graph's own node set, `heads` heads (d / heads in {16, 32, 64});
- * 0 = none (default).  Kernel path 0, inference only (training returns OCCU_EINVAL); with
- * OCCU_BF16 the layers run in FP32 on the BF16-stored h_L (R41); graphormer in [0, 4]. */
+ * 0 = none (default).  Kernel path 0; training in OCCU_FP32 (R47); with OCCU_BF16 inference
+ * runs the layers in FP32 on the BF16-stored h_L (R41) and training returns OCCU_EINVAL;
+ * graphormer in [0, 4]. */
 typedef struct {
   int32_t L, F_n, F_e, d, d_h;
   int32_t aggr;      /* occu_aggr */

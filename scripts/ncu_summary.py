@@ -23,6 +23,9 @@ OUT = os.environ.get("PROFILES_OUT", os.path.join(ROOT, "profiles"))
 
 def kname(full):
     import re
+    m = re.search(r"rowgemm_pair_kernel<(?:\(int\))?(\d+)>", full)
+    if m:
+        return ["node_tc", "edge_tc", "gate_tc"][int(m.group(1))]
     m = re.search(r"rowgemm(?:_bf16)?_kernel<(?:\(int\))?(\d+), (?:\(int\))?(\d+)", full)
     if m:
         return ["node_tc", "edge_tc", "gate_tc", "plain_tc", "gatebwd_tc", "edgebwd_tc",
@@ -32,7 +35,8 @@ def kname(full):
               "head_bwd_reduce", "adam", "wimage", "readout_head", "attn_bwd_q", "attn_bwd_kv",
               "ln_bwd", "colsum", "col_reduce", "mask_dA", "dec_tail_bwd", "dec_pool_bwd",
               "dec_seed_grads", "gph_attn", "gph_ln", "set_decoder_pool", "set_decoder_prep",
-              "set_decoder_kernel", "synth", "wgrad_skinny", "wgrad_partial"):
+              "set_decoder_kernel", "synth", "wgrad_skinny", "wgrad_partial", "row_exp",
+              "gather_hubs", "hub_partial", "hub_merge", "small_forward", "edge_gate", "edgegate"):
         if k in full:
             return k
     return full[:40]
@@ -43,10 +47,16 @@ def launches(tag, path):
     rows = list(csv.reader(io.StringIO(txt[txt.index('"ID"'):])))
     hdr = rows[0]
     iK, iM, iV, iID = hdr.index("Kernel Name"), hdr.index("Metric Name"), hdr.index("Metric Value"), hdr.index("ID")
+    iU = hdr.index("Metric Unit") if "Metric Unit" in hdr else None
+    to_base = {"nsecond": 1.0, "ns": 1.0, "usecond": 1e3, "us": 1e3, "msecond": 1e6, "ms": 1e6,
+               "second": 1e9, "s": 1e9, "byte": 1.0, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9}
     per = collections.OrderedDict()
     for r in rows[1:]:
+        if len(r) <= max(iK, iM, iV, iID):
+            continue
         d = per.setdefault(r[iID], {"kernel": r[iK]})
-        d[r[iM]] = float(r[iV].replace(",", ""))
+        sc = to_base.get(r[iU], 1.0) if iU is not None else 1.0      # times -> ns, bytes -> B
+        d[r[iM]] = float(r[iV].replace(",", "")) * sc
     with open(os.path.join(OUT, f"{tag}_launches.csv"), "w") as f:
         f.write("id,kernel,class,gpu_time_ns,dram_read_bytes,dram_write_bytes\n")
         for i, d in per.items():
@@ -59,9 +69,14 @@ def launches(tag, path):
         a[1] += d.get("gpu__time_duration.sum", 0)
         a[2] += d.get("dram__bytes_read.sum", 0) + d.get("dram__bytes_write.sum", 0)
     tot = sum(a[1] for a in agg.values()) or 1
-    lines = ["| class | launches | share of time | mean DRAM MB / launch |", "|---|---|---|---|"]
+    dram = any(a[2] > 0 for a in agg.values())
+    if dram:
+        lines = ["| class | launches | total µs | share of time | mean DRAM MB / launch |", "|---|---|---|---|---|"]
+    else:
+        lines = ["| class | launches | total µs | share of time |", "|---|---|---|---|"]
     for k, a in sorted(agg.items(), key=lambda x: -x[1][1]):
-        lines.append(f"| {k} | {a[0]} | {100 * a[1] / tot:.1f} % | {a[2] / a[0] / 1e6:.1f} |")
+        row = f"| {k} | {a[0]} | {a[1] / 1e3:.1f} | {100 * a[1] / tot:.1f} % |"
+        lines.append(row + (f" {a[2] / a[0] / 1e6:.1f} |" if dram else ""))
     return "\n".join(lines)
 
 
