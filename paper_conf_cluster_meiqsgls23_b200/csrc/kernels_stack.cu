@@ -11,7 +11,8 @@
 //     dT = (dout W2) ⊙ [T > 0]; dX2 = dT W1; dh̄ = dout + LN2ᵀ(dX2); dO = dh̄ W_o;
 //     attention backward per graph and head (below); dX1 = dQ W_q + dK W_k + dV W_v;
 //     dH = dh̄ + LN1ᵀ(dX1).
-//   Attention backward (FP32 CUDA cores, no atomics): stats m_i, l_i of every query row over
+//   Attention backward (no atomics; tensor cores for d_h in {16, 32}, the FP32 CUDA-core
+//   kernels below for d_h = 64 or with OCCU_ATTN_BWD_SIMT=1): stats m_i, l_i of every query row over
 //   its own graph's keys and D_i = Σ_j P_ij (dO_i·V_j) (= <dO_i, O_i>, from the recomputed P,
 //   taken relative to the dominant key so that saturated softmax rows do not cancel);
 //     dQ_i = Σ_j P_ij (dO_i·V_j − D_i) K_j / √d_h        (thread = query row)
@@ -385,6 +386,345 @@ __global__ void __launch_bounds__(ABT) attn_bwd_kv_kernel(const AttnBwdArgs a) {
   }
 }
 
+
+// ---------------------------------------------------------------------------------------
+// Attention backward on tensor cores (d_h in {16, 32}): the same sums as the CUDA-core kernels
+// above (stats, D' relative to the dominant key, dQ; then dK, dV), every product on mma.sync
+// m16n8k8 TF32 in the 3-product split (x = hi + lo, hi·hi + hi·lo + lo·hi: ~2^-22 relative,
+// the FP32 tolerance; TF32 keeps FP32's exponent range, so the small gradient values need
+// no scaling).  CTA = 64 rows (4 warps x 16) of one head; the other side's rows stream
+// through shared memory in 64-row blocks, pre-split into hi / lo tiles.  The accumulator
+// fragment of S / dP (rows g, g+8; columns 2t, 2t+1 of an 8-wide group) becomes the A operand
+// of the next product without shuffles by reading its k index t as column 2t and t + 4 as
+// column 2t + 1 (the B rows are read in the same order).  Sums over the quad's four threads
+// (softmax stats, D') are combined by xor shuffles (commutative: the same bits on every
+// thread).  No atomics: dQ on the query side, dK / dV on the key side.
+constexpr int MBQ = 64;               // rows per CTA (4 warps x 16)
+constexpr int MBK = 64;               // rows per staged block
+
+// x = hi + lo with hi = x rounded to tf32 (round half away on the magnitude: the integer form
+// of cvt.rna.tf32.f32 for finite x, which ptxas expands with an Inf/NaN guard) and lo = x − hi
+// exactly; the MMA truncates lo to tf32, an error <= 2^-11·|lo| <= 2^-22·|x|.
+__device__ __forceinline__ void tf32_split(float x, uint32_t &hi, uint32_t &lo) {
+  const uint32_t h = (__float_as_uint(x) + 0x1000u) & 0xFFFFE000u;
+  hi = h;
+  lo = __float_as_uint(x - __uint_as_float(h));
+}
+__device__ __forceinline__ void mma_tf32(float (&c)[4], const uint32_t (&a)[4], uint32_t b0, uint32_t b1) {
+  asm volatile(
+      "mma.sync.aligned.m16n8k8.row.col.f32.tf32.tf32.f32 {%0,%1,%2,%3}, {%4,%5,%6,%7}, {%8,%9}, "
+      "{%0,%1,%2,%3};"
+      : "+f"(c[0]), "+f"(c[1]), "+f"(c[2]), "+f"(c[3])
+      : "r"(a[0]), "r"(a[1]), "r"(a[2]), "r"(a[3]), "r"(b0), "r"(b1));
+}
+// rows [r0, r0 + MBK) of X (head slice, times sc) -> hi / lo tiles [MBK][DH + 4]; every
+// thread issues all of its float4 loads before the first split (latency overlapped)
+template <int DH>
+__device__ __forceinline__ void stage_split(const float *__restrict__ X, int D, int hc, int r0, int r1,
+                                            float sc, float *xh, float *xl) {
+  constexpr int SR = DH + 4, C4 = DH / 4, PER = MBK * C4 / 128;
+  float4 v[PER];
+#pragma unroll
+  for (int u = 0; u < PER; ++u) {
+    const int e = threadIdx.x + 128 * u, rr = e / C4, c4 = (e % C4) * 4;
+    v[u] = r0 + rr < r1 ? __ldg(reinterpret_cast<const float4 *>(X + long(r0 + rr) * D + hc + c4))
+                        : make_float4(0.f, 0.f, 0.f, 0.f);
+  }
+#pragma unroll
+  for (int u = 0; u < PER; ++u) {
+    const int e = threadIdx.x + 128 * u, rr = e / C4, c4 = (e % C4) * 4;
+    const float x[4] = {v[u].x * sc, v[u].y * sc, v[u].z * sc, v[u].w * sc};
+    uint32_t hi[4], lo[4];
+#pragma unroll
+    for (int k = 0; k < 4; ++k) tf32_split(x[k], hi[k], lo[k]);
+    *reinterpret_cast<uint4 *>(xh + rr * SR + c4) = make_uint4(hi[0], hi[1], hi[2], hi[3]);
+    *reinterpret_cast<uint4 *>(xl + rr * SR + c4) = make_uint4(lo[0], lo[1], lo[2], lo[3]);
+  }
+}
+// A fragment (16 rows x 8 columns at column c0) of rows ra / rb of X (head slice, times sc)
+__device__ __forceinline__ void frag_a(const float *__restrict__ X, int D, int hc, long ra, long rb, int N,
+                                       int c0, int t, float sc, uint32_t (&h)[4], uint32_t (&l)[4]) {
+#pragma unroll
+  for (int q = 0; q < 4; ++q) {
+    const long r = (q & 1) ? rb : ra;
+    const int c = c0 + t + (q >> 1) * 4;
+    const float x = r < N ? __ldg(X + r * D + hc + c) * sc : 0.f;
+    tf32_split(x, h[q], l[q]);
+  }
+}
+constexpr float LOG2E_F = 1.4426950408889634f;
+__device__ __forceinline__ float ex2a(float x) {
+  float r;
+  asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(r) : "f"(x));
+  return r;
+}
+constexpr int MNG = 4;                // 8-row groups processed together (independent MMA chains)
+
+// S (or dP) of MNG consecutive 8-column groups starting at block row nt0, A fragments a*[KS],
+// B rows from the staged hi / lo tile: per ks the MNG groups' MMAs interleave (independent
+// accumulators) so the tensor pipe is not serialised on one accumulator.
+template <int KS, int SR>
+__device__ __forceinline__ void prod_groups(float (&c)[MNG][4], const uint32_t (&ah)[KS][4], const uint32_t (&al)[KS][4],
+                                            const float *bh, const float *bl, int nt0, int g, int t) {
+#pragma unroll
+  for (int q = 0; q < MNG; ++q) c[q][0] = c[q][1] = c[q][2] = c[q][3] = 0.f;
+#pragma unroll
+  for (int ks = 0; ks < KS; ++ks) {
+#pragma unroll
+    for (int q = 0; q < MNG; ++q) {
+      const int o = (nt0 + 8 * q + g) * SR + ks * 8 + t;
+      mma_tf32(c[q], ah[ks], __float_as_uint(bh[o]), __float_as_uint(bh[o + 4]));
+    }
+#pragma unroll
+    for (int q = 0; q < MNG; ++q) {
+      const int o = (nt0 + 8 * q + g) * SR + ks * 8 + t;
+      mma_tf32(c[q], ah[ks], __float_as_uint(bl[o]), __float_as_uint(bl[o + 4]));
+    }
+#pragma unroll
+    for (int q = 0; q < MNG; ++q) {
+      const int o = (nt0 + 8 * q + g) * SR + ks * 8 + t;
+      mma_tf32(c[q], al[ks], __float_as_uint(bh[o]), __float_as_uint(bh[o + 4]));
+    }
+  }
+}
+// C fragment (rows g / g+8, columns 2t / 2t+1 of an 8-wide group) -> A fragment with k = t as
+// column 2t and k = t + 4 as column 2t + 1, split hi / lo
+__device__ __forceinline__ void c_to_a(const float (&c)[4], uint32_t (&h)[4], uint32_t (&l)[4]) {
+  tf32_split(c[0], h[0], l[0]);
+  tf32_split(c[2], h[1], l[1]);
+  tf32_split(c[1], h[2], l[2]);
+  tf32_split(c[3], h[3], l[3]);
+}
+// acc[n] += A (16 x 8, from c_to_a) x B (8 staged rows nt+2t / nt+2t+1 read as k, columns n·8 + g)
+template <int NO, int SR>
+__device__ __forceinline__ void prod_rows(float (&acc)[NO][4], const uint32_t (&h)[4], const uint32_t (&l)[4],
+                                          const float *bh, const float *bl, int nt, int g, int t) {
+#pragma unroll
+  for (int n = 0; n < NO; ++n) {
+    const int o0 = (nt + 2 * t) * SR + n * 8 + g, o1 = o0 + SR;
+    mma_tf32(acc[n], h, __float_as_uint(bh[o0]), __float_as_uint(bh[o1]));
+  }
+#pragma unroll
+  for (int n = 0; n < NO; ++n) {
+    const int o0 = (nt + 2 * t) * SR + n * 8 + g, o1 = o0 + SR;
+    mma_tf32(acc[n], h, __float_as_uint(bl[o0]), __float_as_uint(bl[o1]));
+  }
+#pragma unroll
+  for (int n = 0; n < NO; ++n) {
+    const int o0 = (nt + 2 * t) * SR + n * 8 + g, o1 = o0 + SR;
+    mma_tf32(acc[n], l, __float_as_uint(bh[o0]), __float_as_uint(bh[o1]));
+  }
+}
+
+__device__ __forceinline__ void quad_merge2(float &m, float &l, int &ref) {
+#pragma unroll
+  for (int o = 1; o <= 2; o <<= 1) {
+    const float m2 = __shfl_xor_sync(0xffffffffu, m, o);
+    const float l2 = __shfl_xor_sync(0xffffffffu, l, o);
+    const int r2 = __shfl_xor_sync(0xffffffffu, ref, o);
+    const float mm = fmaxf(m, m2);
+    if (mm == -INFINITY) continue;
+    const float nl = (m == -INFINITY ? 0.f : l * ex2a(m - mm)) + (m2 == -INFINITY ? 0.f : l2 * ex2a(m2 - mm));
+    const int nr = (m == mm && m2 == mm) ? min(ref, r2) : (m2 == mm ? r2 : ref);
+    m = mm;
+    l = nl;
+    ref = nr;
+  }
+}
+
+template <int DH>
+__global__ void __launch_bounds__(128) attn_bwd_q_mma_kernel(const AttnBwdArgs a) {
+  constexpr int KS = DH / 8, NO = DH / 8, SR = DH + 4;
+  extern __shared__ float smq[];
+  float *Kh = smq, *Kl = Kh + MBK * SR, *Vh = Kl + MBK * SR, *Vl = Vh + MBK * SR;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, g = lane >> 2, t = lane & 3;
+  const int h = blockIdx.y, hc = h * DH, D = a.D;
+  const long q0 = long(blockIdx.x) * MBQ;
+  const long qlast = min(q0 + MBQ, long(a.N)) - 1;
+  const int ub = __ldg(a.node_off + __ldg(a.node_graph + q0));
+  const int ue = __ldg(a.node_off + __ldg(a.node_graph + qlast) + 1);
+  const long ra = q0 + warp * 16 + g, rb = ra + 8;
+  int kla = 0, kha = 0, klb = 0, khb = 0;
+  if (ra < a.N) { const int b = __ldg(a.node_graph + ra); kla = __ldg(a.node_off + b); kha = __ldg(a.node_off + b + 1); }
+  if (rb < a.N) { const int b = __ldg(a.node_graph + rb); klb = __ldg(a.node_off + b); khb = __ldg(a.node_off + b + 1); }
+  // Q carries log2(e)/√d_h: scores come out in log2 units for ex2
+  uint32_t qh[KS][4], ql[KS][4], oh[KS][4], ol[KS][4];
+#pragma unroll
+  for (int ks = 0; ks < KS; ++ks) {
+    frag_a(a.Q, D, hc, ra, rb, a.N, ks * 8, t, a.scale * LOG2E_F, qh[ks], ql[ks]);
+    frag_a(a.dO, D, hc, ra, rb, a.N, ks * 8, t, 1.f, oh[ks], ol[ks]);
+  }
+  auto inrow = [&](int e, int j) { return (e < 2) ? (j >= kla && j < kha) : (j >= klb && j < khb); };
+  // pass 1: row maximum (first arg max) and normaliser over the own graph's keys (log2 units)
+  float ma = -INFINITY, mb = -INFINITY, la = 0.f, lb = 0.f;
+  int refa = kla, refb = klb;
+  for (int t0 = ub; t0 < ue; t0 += MBK) {
+    __syncthreads();
+    stage_split<DH>(a.K, D, hc, t0, ue, 1.f, Kh, Kl);
+    __syncthreads();
+    for (int nt0 = 0; nt0 < MBK && t0 + nt0 < ue; nt0 += 8 * MNG) {
+      float s[MNG][4];
+      prod_groups<KS, SR>(s, qh, ql, Kh, Kl, nt0, g, t);
+#pragma unroll
+      for (int q = 0; q < MNG; ++q)
+#pragma unroll
+        for (int e = 0; e < 4; ++e) {
+          const int j = t0 + nt0 + 8 * q + 2 * t + (e & 1);
+          float &m = (e < 2) ? ma : mb;
+          float &l = (e < 2) ? la : lb;
+          int &ref = (e < 2) ? refa : refb;
+          if (inrow(e, j)) {
+            if (s[q][e] > m) {
+              l = (m == -INFINITY ? 0.f : l * ex2a(m - s[q][e])) + 1.f;
+              m = s[q][e];
+              ref = j;
+            } else {
+              l += ex2a(s[q][e] - m);
+            }
+          }
+        }
+    }
+  }
+  quad_merge2(ma, la, refa);
+  quad_merge2(mb, lb, refb);
+  const float ila = la > 0.f ? 1.f / la : 0.f, ilb = lb > 0.f ? 1.f / lb : 0.f;
+  float dpra = 0.f, dprb = 0.f;                        // dP_ir against the dominant key
+  if (ra < a.N)
+    for (int c = 0; c < DH; ++c) dpra = fmaf(__ldg(a.dO + ra * D + hc + c), __ldg(a.V + long(refa) * D + hc + c), dpra);
+  if (rb < a.N)
+    for (int c = 0; c < DH; ++c) dprb = fmaf(__ldg(a.dO + rb * D + hc + c), __ldg(a.V + long(refb) * D + hc + c), dprb);
+  // pass 2: D'_i = Σ_j P_ij (dP_ij − dP_ir) (float64); pass 3: dQ_i = Σ_j dS_ij K_j
+  double Da = 0.0, Db = 0.0;
+  float Dpa = 0.f, Dpb = 0.f;
+  float dq[NO][4];
+#pragma unroll
+  for (int n = 0; n < NO; ++n) dq[n][0] = dq[n][1] = dq[n][2] = dq[n][3] = 0.f;
+  for (int pass = 2; pass <= 3; ++pass) {
+    for (int t0 = ub; t0 < ue; t0 += MBK) {
+      __syncthreads();
+      stage_split<DH>(a.K, D, hc, t0, ue, 1.f, Kh, Kl);
+      stage_split<DH>(a.V, D, hc, t0, ue, 1.f, Vh, Vl);
+      __syncthreads();
+      for (int nt0 = 0; nt0 < MBK && t0 + nt0 < ue; nt0 += 8 * MNG) {
+        float s[MNG][4], dp[MNG][4];
+        prod_groups<KS, SR>(s, qh, ql, Kh, Kl, nt0, g, t);
+        prod_groups<KS, SR>(dp, oh, ol, Vh, Vl, nt0, g, t);
+#pragma unroll
+        for (int q = 0; q < MNG; ++q) {
+          float ds[4];
+#pragma unroll
+          for (int e = 0; e < 4; ++e) {
+            const int j = t0 + nt0 + 8 * q + 2 * t + (e & 1);
+            const float p = inrow(e, j) ? ex2a(s[q][e] - (e < 2 ? ma : mb)) * (e < 2 ? ila : ilb) : 0.f;
+            const float dd = dp[q][e] - (e < 2 ? dpra : dprb);
+            if (pass == 2) {
+              if (e < 2) Da = fma(double(p), double(dd), Da);
+              else Db = fma(double(p), double(dd), Db);
+            }
+            ds[e] = p * (dd - (e < 2 ? Dpa : Dpb));
+          }
+          if (pass == 3) {
+            uint32_t dh_[4], dl_[4];
+            c_to_a(ds, dh_, dl_);
+            prod_rows<NO, SR>(dq, dh_, dl_, Kh, Kl, nt0 + 8 * q, g, t);
+          }
+        }
+      }
+    }
+    if (pass == 2) {
+#pragma unroll
+      for (int o = 1; o <= 2; o <<= 1) {
+        Da += __shfl_xor_sync(0xffffffffu, Da, o);
+        Db += __shfl_xor_sync(0xffffffffu, Db, o);
+      }
+      Dpa = float(Da);
+      Dpb = float(Db);
+    }
+  }
+#pragma unroll
+  for (int n = 0; n < NO; ++n) {
+    const int c = hc + n * 8 + 2 * t;
+    if (ra < a.N) *reinterpret_cast<float2 *>(a.dQ + ra * D + c) = make_float2(dq[n][0] * a.scale, dq[n][1] * a.scale);
+    if (rb < a.N) *reinterpret_cast<float2 *>(a.dQ + rb * D + c) = make_float2(dq[n][2] * a.scale, dq[n][3] * a.scale);
+  }
+  if (t == 0) {               // stats in log2 units (m), as the key-side kernel reads them
+    if (ra < a.N) *reinterpret_cast<float4 *>(a.stats + (ra * a.heads + h) * 4) = make_float4(ma, la, Dpa, dpra);
+    if (rb < a.N) *reinterpret_cast<float4 *>(a.stats + (rb * a.heads + h) * 4) = make_float4(mb, lb, Dpb, dprb);
+  }
+}
+
+template <int DH>
+__global__ void __launch_bounds__(128) attn_bwd_kv_mma_kernel(const AttnBwdArgs a) {
+  constexpr int KS = DH / 8, NO = DH / 8, SR = DH + 4;
+  extern __shared__ float smk[];
+  float *Qh = smk, *Ql = Qh + MBK * SR, *Oh = Ql + MBK * SR, *Ol = Oh + MBK * SR;
+  float4 *ss = reinterpret_cast<float4 *>(Ol + MBK * SR);     // [MBK] m (log2), l, D', dP_ir
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, g = lane >> 2, t = lane & 3;
+  const int h = blockIdx.y, hc = h * DH, D = a.D;
+  const long j0 = long(blockIdx.x) * MBQ;
+  const long jlast = min(j0 + MBQ, long(a.N)) - 1;
+  const int ub = __ldg(a.node_off + __ldg(a.node_graph + j0));
+  const int ue = __ldg(a.node_off + __ldg(a.node_graph + jlast) + 1);
+  const long ja = j0 + warp * 16 + g, jb = ja + 8;
+  int qla = 0, qha = 0, qlb = 0, qhb = 0;
+  if (ja < a.N) { const int b = __ldg(a.node_graph + ja); qla = __ldg(a.node_off + b); qha = __ldg(a.node_off + b + 1); }
+  if (jb < a.N) { const int b = __ldg(a.node_graph + jb); qlb = __ldg(a.node_off + b); qhb = __ldg(a.node_off + b + 1); }
+  uint32_t kh[KS][4], kl[KS][4], vh[KS][4], vl[KS][4];
+#pragma unroll
+  for (int ks = 0; ks < KS; ++ks) {
+    frag_a(a.K, D, hc, ja, jb, a.N, ks * 8, t, 1.f, kh[ks], kl[ks]);
+    frag_a(a.V, D, hc, ja, jb, a.N, ks * 8, t, 1.f, vh[ks], vl[ks]);
+  }
+  float dk[NO][4], dv[NO][4];
+#pragma unroll
+  for (int n = 0; n < NO; ++n) dk[n][0] = dk[n][1] = dk[n][2] = dk[n][3] = dv[n][0] = dv[n][1] = dv[n][2] = dv[n][3] = 0.f;
+  for (int t0 = ub; t0 < ue; t0 += MBK) {
+    __syncthreads();
+    stage_split<DH>(a.Q, D, hc, t0, ue, a.scale * LOG2E_F, Qh, Ql);     // scores in log2 units
+    stage_split<DH>(a.dO, D, hc, t0, ue, 1.f, Oh, Ol);
+    for (int e = threadIdx.x; e < MBK; e += 128)
+      ss[e] = t0 + e < ue ? *reinterpret_cast<const float4 *>(a.stats + (long(t0 + e) * a.heads + h) * 4)
+                          : make_float4(0.f, 1.f, 0.f, 0.f);
+    __syncthreads();
+    for (int nt0 = 0; nt0 < MBK && t0 + nt0 < ue; nt0 += 8 * MNG) {
+      // Sᵀ, dPᵀ of the query groups: c0 (ja, query 2t), c1 (ja, 2t+1), c2 (jb, 2t), c3 (jb, 2t+1)
+      float s[MNG][4], dp[MNG][4];
+      prod_groups<KS, SR>(s, kh, kl, Qh, Ql, nt0, g, t);
+      prod_groups<KS, SR>(dp, vh, vl, Oh, Ol, nt0, g, t);
+#pragma unroll
+      for (int q = 0; q < MNG; ++q) {
+        float p[4], ds[4];
+#pragma unroll
+        for (int e = 0; e < 4; ++e) {
+          const int qi = nt0 + 8 * q + 2 * t + (e & 1), i = t0 + qi;
+          const bool in = (e < 2) ? (i >= qla && i < qha) : (i >= qlb && i < qhb);
+          const float4 st = ss[qi];
+          p[e] = in ? ex2a(s[q][e] - st.x) / st.y : 0.f;
+          ds[e] = p[e] * ((dp[q][e] - st.w) - st.z);
+        }
+        uint32_t ph[4], pl[4], dh_[4], dl_[4];
+        c_to_a(p, ph, pl);
+        c_to_a(ds, dh_, dl_);
+        prod_rows<NO, SR>(dv, ph, pl, Oh, Ol, nt0 + 8 * q, g, t);
+        prod_rows<NO, SR>(dk, dh_, dl_, Qh, Ql, nt0 + 8 * q, g, t);
+      }
+    }
+  }
+  // Qh carried log2(e)/√d_h; dK = Σ dS Q/√d_h
+  const float kfix = 1.f / LOG2E_F;
+#pragma unroll
+  for (int n = 0; n < NO; ++n) {
+    const int c = hc + n * 8 + 2 * t;
+    if (ja < a.N) {
+      *reinterpret_cast<float2 *>(a.dK + ja * D + c) = make_float2(dk[n][0] * kfix, dk[n][1] * kfix);
+      *reinterpret_cast<float2 *>(a.dV + ja * D + c) = make_float2(dv[n][0], dv[n][1]);
+    }
+    if (jb < a.N) {
+      *reinterpret_cast<float2 *>(a.dK + jb * D + c) = make_float2(dk[n][2] * kfix, dk[n][3] * kfix);
+      *reinterpret_cast<float2 *>(a.dV + jb * D + c) = make_float2(dv[n][2], dv[n][3]);
+    }
+  }
+}
 }  // namespace
 
 // ---- launchers ---------------------------------------------------------------------------
@@ -483,8 +823,19 @@ int launch_graphormer_layer_bwd(occu_ctx *ctx, const DevCsr &csr, int j, const f
   const int dh = D / cf.heads;
   a.scale = 1.f / sqrtf(float(dh));
   const dim3 grid((N + ABT - 1) / ABT, cf.heads);
+  static const bool simt_attn = getenv("OCCU_ATTN_BWD_SIMT") != nullptr;   // A/B: CUDA-core kernels
   OCCU_PROF_BEGIN(ctx, "stack_attn_bwd", st);
-  switch (dh) {
+  if (!simt_attn && (dh == 16 || dh == 32)) {
+    const dim3 mg((N + MBQ - 1) / MBQ, cf.heads);
+    const size_t smq = size_t(4) * MBK * (dh + 4) * 4, smk = smq + size_t(MBK) * 16;
+    if (dh == 16) {
+      attn_bwd_q_mma_kernel<16><<<mg, 128, smq, st>>>(a);
+      attn_bwd_kv_mma_kernel<16><<<mg, 128, smk, st>>>(a);
+    } else {
+      attn_bwd_q_mma_kernel<32><<<mg, 128, smq, st>>>(a);
+      attn_bwd_kv_mma_kernel<32><<<mg, 128, smk, st>>>(a);
+    }
+  } else switch (dh) {
     case 16: attn_bwd_q_kernel<16><<<grid, ABT, 0, st>>>(a); attn_bwd_kv_kernel<16><<<grid, ABT, 0, st>>>(a); break;
     case 32: attn_bwd_q_kernel<32><<<grid, ABT, 0, st>>>(a); attn_bwd_kv_kernel<32><<<grid, ABT, 0, st>>>(a); break;
     case 64: attn_bwd_q_kernel<64><<<grid, ABT, 0, st>>>(a); attn_bwd_kv_kernel<64><<<grid, ABT, 0, st>>>(a); break;
