@@ -891,6 +891,13 @@ class Bench:
         best = min(v for k, v in det.items() if k.endswith("_us"))
         self.put("cfg1_latency_us", best, "f32", det, unit="us/graph")
 
+    def _templates(self, m, fams=None):
+        from occu_gen import configs
+        from occu_gen import templates as tmpl_mod
+        if not hasattr(self, "_host_tmpl"):
+            self._host_tmpl = {f: tmpl_mod.build_template(f) for f in configs.MIXTURE}
+        return [m.template(self._host_tmpl[f]) for f in (fams or configs.MIXTURE)]
+
     def sec_cfg4(self):
         """CFG4: the FULL 50,000-graph data-parallel training epoch on the 20-family mixture.
         Every step's global micro-batch of 256 x N graphs is LPT-sharded over the ranks by
