@@ -680,8 +680,14 @@ class Bench:
                 "achieved": flops / (ams * 1e-3) / 1e12, "peak": peak, "unit": "TFLOP/s",
                 "frac": flops / (ams * 1e-3) / 1e12 / peak,
                 "peak_kind": "measured bf16 dense (= fp16 kind::f16) / 3 products (fp16x2 split)"}
-        det["bf16"] = "unavailable: d = 256 runs OCCU_FP32 only in this build"
         del m, csr
+        mb = self.model(L=1, d=d, prec=self.occu.BF16)
+        mb.init_weights(42)
+        csr = mb.to_device(self.cfg2_host_csr)
+        alg2 = algorithmic_bytes(N, E, B, d=d, L=1, rrows=readout_rows(b.graphs), sa=2)
+        ms2, _, _ = self._infer("cfg2_paper_bf16", mb, csr, nf, ef, B, alg2, "bf16")
+        self.details["cfg2_paper_bf16"]["survey_step_bytes"] = survey_step_bytes(N, E, B, d=d, L=1, sa=2)
+        del mb, csr
 
     def sec_cfg2_train(self):
         occu, torch = self.occu, self.torch

@@ -60,10 +60,10 @@ typedef enum { OCCU_FP32 = 0, OCCU_BF16 = 1 } occu_precision;
 typedef enum { OCCU_READOUT_MEAN = 0, OCCU_READOUT_SET_DECODER = 1 } occu_readout;
 
 /* Model configuration.  L ANEE rounds of width d (64, 128 or 256); d = 256 is the paper's
- * hidden width (P273) and runs on the CTA-pair tensor-core path: OCCU_FP32,
- * msg = OCCU_MSG_CHANNEL_SOFTMAX, readout MEAN, graphormer = 0, F_n <= 256, inference only
- * (occu_train_step / occu_grads return OCCU_EINVAL; any other d, or d = 256 with another
- * mode, fails occu_create with OCCU_EINVAL).  Raw feature
+ * hidden width (P273) and runs on the CTA-pair tensor-core path: OCCU_FP32 or
+ * OCCU_BF16 (BF16: F_e <= 16), msg = OCCU_MSG_CHANNEL_SOFTMAX, readout MEAN, graphormer = 0,
+ * F_n <= 256, inference only (occu_train_step / occu_grads return OCCU_EINVAL; any other d,
+ * or d = 256 with another mode, fails occu_create with OCCU_EINVAL).  Raw feature
  * widths F_n (node, Table I) and F_e (edge); head hidden width d_h; LeakyReLU slope (R7,
  * 0.01); F_n, F_e multiples of 4.  msg = OCCU_MSG_NEIGHBOR_SOFTMAX (reading B, NEXT-1):
  * kernel path 0; OCCU_FP32 forward + training, OCCU_BF16 forward (training with OCCU_BF16

@@ -499,7 +499,8 @@ __global__ void __launch_bounds__(256) edge_small_bf16_kernel(
         o[v / 2] = pack_bf16(fast_rcp(1.f + ex2(-(a * z[v]) * LOG2E)),
                              fast_rcp(1.f + ex2(-(a * z[v + 1]) * LOG2E)));
       __nv_bfloat16 *dst = e_out + (k0 + u) * D + c;
-      if constexpr (V == 4) *reinterpret_cast<uint2 *>(dst) = make_uint2(o[0], o[1]);
+      if constexpr (V == 8) *reinterpret_cast<uint4 *>(dst) = make_uint4(o[0], o[1 % (V / 2)], o[2 % (V / 2)], o[3 % (V / 2)]);
+      else if constexpr (V == 4) *reinterpret_cast<uint2 *>(dst) = make_uint2(o[0], o[1 % (V / 2)]);
       else *reinterpret_cast<uint32_t *>(dst) = o[0];
     }
   }
@@ -643,11 +644,50 @@ int launch_bwd_edge_bf16(const occu_ctx *ctx, const DevCsr &csr, int layer, cons
   }
 }
 
+// d = 256 in OCCU_BF16: the three row-GEMMs on CTA pairs (launch_pair_bf16, kernels_tc.cu),
+// the layer-1 edge transform and the aggregation as at d <= 128
+static int forward_layer_bf16_256(const occu_ctx *ctx, const DevCsr &csr, int layer, const FwdLayerArgs &a,
+                                  cudaStream_t st) {
+  constexpr int D = 256;
+  if (ctx->cfg.msg != OCCU_MSG_CHANNEL_SOFTMAX) return -int(cudaErrorInvalidValue);
+  int n = 0, r;
+  if ((r = launch_pair_bf16(ctx, 0, layer == 0, a.h_in, a.K, csr.N, layer, a.hbar, a.a_s, a.a_d, a.p, a.q,
+                            nullptr, nullptr, "node_tc", st)) < 0) return r;
+  n += r;
+  if (csr.E > 0) {
+    __nv_bfloat16 *e_out = reinterpret_cast<__nv_bfloat16 *>(a.e_out);
+    if (a.Ke <= 16) {
+      const int grid = int(std::min<long>((long(csr.E) + 255) / 256, 8L * ctx->num_sms));
+      OCCU_PROF_BEGIN(ctx, "edge_small", st);
+      if (a.Ke <= 4)
+        launch_pdl(ctx->pdl & 4, edge_small_bf16_kernel<D, 4>, grid, 256, D * a.Ke * 4, st, a.e_in, a.Ke,
+                   a.W_e, a.p, a.q, csr.in_src, csr.in_dst, a.e_eid, csr.E, e_out, a.e0_out);
+      else
+        launch_pdl(ctx->pdl & 4, edge_small_bf16_kernel<D, 16>, grid, 256, D * a.Ke * 4, st, a.e_in, a.Ke,
+                   a.W_e, a.p, a.q, csr.in_src, csr.in_dst, a.e_eid, csr.E, e_out, a.e0_out);
+      OCCU_PROF_END(ctx);
+      const cudaError_t e = cudaGetLastError();
+      if (e != cudaSuccess) return -int(e);
+      ++n;
+    } else {
+      if ((r = launch_pair_bf16(ctx, 1, layer == 0, a.e_in, a.Ke, csr.E, layer, e_out, nullptr, nullptr,
+                                a.p, a.q, csr.in_src, csr.in_dst, "edge_tc", st)) < 0) return r;
+      n += r;
+    }
+    if ((r = launch_pair_bf16(ctx, 2, false, a.e_out, D, csr.E, layer, a.g, nullptr, nullptr, nullptr,
+                              nullptr, nullptr, nullptr, "gate_tc", st)) < 0) return r;
+    n += r;
+  }
+  if ((r = launch_gather_segsum_bf16(ctx, csr, a.g, a.hbar, a.h_out, a.rpart, st)) < 0) return r;
+  return n + r;
+}
+
 int launch_forward_layer_bf16(const occu_ctx *ctx, const DevCsr &csr, int layer,
                               const FwdLayerArgs &a, cudaStream_t st) {
   switch (ctx->cfg.d) {
     case 64: return forward_layer_bf16<64>(ctx, csr, layer, a, st);
     case 128: return forward_layer_bf16<128>(ctx, csr, layer, a, st);
+    case 256: return forward_layer_bf16_256(ctx, csr, layer, a, st);
     default: return -int(cudaErrorInvalidValue);
   }
 }

@@ -2026,7 +2026,10 @@ static int gather_bf16_impl(const occu_ctx *ctx, const DevCsr &csr, const void *
   if (r0 < 0) return r0;
   OCCU_PROF_BEGIN(ctx, "gather_segsum", st);
 #define OCCU_GB_ARGS g, hbar, csr.in_ptr, csr.in_src, csr.N, mean, ctx->cfg.slope, h_out, csr.node_graph, rpart, hub, csr.in_dst
-  if (gsel == 4) {
+  if constexpr (D == 256) {
+    if (rpart) launch_pdl(ctx->pdl & 64, gather_segsum_v2_kernel<D, 2, true, true>, grid, NT, 0, st, OCCU_GB_ARGS);
+    else launch_pdl(ctx->pdl & 64, gather_segsum_v2_kernel<D, 2, false, true>, grid, NT, 0, st, OCCU_GB_ARGS);
+  } else if (gsel == 4) {
     if (rpart) launch_pdl(ctx->pdl & 64, gather_segsum_v2_kernel<D, 4, true, true>, grid, NT, 0, st, OCCU_GB_ARGS);
     else launch_pdl(ctx->pdl & 64, gather_segsum_v2_kernel<D, 4, false, true>, grid, NT, 0, st, OCCU_GB_ARGS);
   } else if (gsel == 2) {
@@ -2087,6 +2090,7 @@ int launch_gather_segsum_bf16(const occu_ctx *ctx, const DevCsr &csr, const void
   switch (ctx->cfg.d) {
     case 64: return gather_bf16_impl<64>(ctx, csr, g, hbar, h_out, rpart, st);
     case 128: return gather_bf16_impl<128>(ctx, csr, g, hbar, h_out, rpart, st);
+    case 256: return gather_bf16_impl<256>(ctx, csr, g, hbar, h_out, rpart, st);
     default: return -int(cudaErrorInvalidValue);
   }
 }

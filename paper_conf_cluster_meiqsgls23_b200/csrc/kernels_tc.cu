@@ -919,20 +919,21 @@ struct PairSmem {
   float *xbuf;                        // 16 epilogue warps x 16 x 20 floats
 };
 
-__host__ __device__ inline size_t pair_smem_bytes(int K) {
+// nimg: 2 fp16x2 images (OCCU_FP32) or 1 BF16 image (OCCU_BF16)
+__host__ __device__ inline size_t pair_smem_bytes(int K, int nimg) {
   const size_t img = size_t(kpad_of(K)) * 128 * 2;
-  return 1024 + 2 * img + size_t(P_NS) * 16384 + 256 + 2048 + 4096 + 16 * 16 * 20 * 4;
+  return 1024 + nimg * img + size_t(P_NS) * 16384 + 256 + 2048 + 4096 + 16 * 16 * 20 * 4;
 }
 
-__device__ __forceinline__ PairSmem carve_pair(uint8_t *raw, int K) {
+__device__ __forceinline__ PairSmem carve_pair(uint8_t *raw, int K, int nimg) {
   PairSmem s;
   const uint32_t a = tc::smem_u32(raw);
   uint8_t *base = raw + ((1024 - (a & 1023)) & 1023);
   const size_t img = size_t(kpad_of(K)) * 128 * 2;
   s.w0 = base;
   s.w1 = base + img;
-  s.ring = reinterpret_cast<float *>(base + 2 * img);
-  uint8_t *misc = base + 2 * img + size_t(P_NS) * 16384;
+  s.ring = reinterpret_cast<float *>(base + nimg * img);
+  uint8_t *misc = base + nimg * img + size_t(P_NS) * 16384;
   uint64_t *bars = reinterpret_cast<uint64_t *>(misc);
   s.full = bars;
   s.empty = bars + P_NS;
@@ -951,12 +952,38 @@ __device__ __forceinline__ PairSmem carve_pair(uint8_t *raw, int K) {
 
 __device__ __forceinline__ void epi_bar_pair() { asm volatile("bar.sync 1, 512;" ::: "memory"); }
 
-template <int EPI>
+__device__ __forceinline__ uint32_t pack_bf16_rn(float x0, float x1) {
+  const __nv_bfloat162 b = __floats2bfloat162_rn(x0, x1);
+  return *reinterpret_cast<const uint32_t *>(&b);
+}
+// 16 channels of the thread's row: FP32 through the coalescing transpose; BF16 as one
+// 32-byte sector per row
+template <bool BF>
+__device__ __forceinline__ void pair_store(float *wbuf, float *out, long wrow0, int wrows, long grow,
+                                           bool live, int c0, const float (&o)[16], int lane) {
+  if (BF) {
+    if (!live) return;
+    uint32_t w[8];
+#pragma unroll
+    for (int u = 0; u < 8; ++u) w[u] = pack_bf16_rn(o[2 * u], o[2 * u + 1]);
+    uint4 *dst = reinterpret_cast<uint4 *>(reinterpret_cast<__nv_bfloat16 *>(out) + grow * PD + c0);
+    dst[0] = make_uint4(w[0], w[1], w[2], w[3]);
+    dst[1] = make_uint4(w[4], w[5], w[6], w[7]);
+  } else {
+    warp_store_chunk<PD>(wbuf, out, wrow0, wrows, c0, o, lane);
+  }
+}
+
+// BF: OCCU_BF16 (one BF16 image, one product per K step, BF16 outputs, no row scale);
+// AF32: the input rows are FP32 (every FP32-mode input; the layer-1 node features in BF16
+// mode), else BF16 rows (TMA boxes of 128 rows x 64 bf16).
+template <int EPI, bool BF, bool AF32>
 __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(P_NTH, 1)
     rowgemm_pair_kernel(const __grid_constant__ CUtensorMap tmap, RowGemmArgs a) {
   extern __shared__ uint8_t smem_raw[];
-  const int K = a.K, Kpad = kpad_of(K), NC = Kpad / 64, NB = nbox_of(K);
-  PairSmem s = carve_pair(smem_raw, K);
+  constexpr int EPB = AF32 ? 32 : 64;                          // K elements per box
+  const int K = a.K, Kpad = kpad_of(K), NC = Kpad / 64, NB = (K + EPB - 1) / EPB;
+  PairSmem s = carve_pair(smem_raw, K, BF ? 1 : 2);
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const uint32_t rank = tc::cluster_rank();
 
@@ -1005,11 +1032,11 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(P_NTH, 1)
     if (lane == 0) {
       tc::prefetch_tmap(&tmap);
       const uint32_t ib = uint32_t(Kpad) * PD * 2;            // one full image (w0 or w1)
-      tc::mbar_arrive_expect_tx(s.wfull, uint32_t(Kpad) * 128u * 2u * 2u);
+      tc::mbar_arrive_expect_tx(s.wfull, uint32_t(Kpad) * 128u * 2u * (BF ? 1u : 2u));
       for (int c = 0; c < NC; ++c) {                          // 16 KB per 64-wide K chunk
         const uint32_t src = uint32_t(c) * 32768u + rank * 16384u;
         tc::bulk_g2s(s.w0 + c * 16384, a.wimg + src, 16384, s.wfull);
-        tc::bulk_g2s(s.w1 + c * 16384, a.wimg + ib + src, 16384, s.wfull);
+        if (!BF) tc::bulk_g2s(s.w1 + c * 16384, a.wimg + ib + src, 16384, s.wfull);
       }
       if (rank == 1) {                                       // tell the leader its B half is in
         tc::mbar_wait(s.wfull, 0);
@@ -1021,7 +1048,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(P_NTH, 1)
       auto prefetch = [&](long qq) {
         if (qq >= nq) return;
         const long rr = row0_of(int(qq / NB));
-        if (rr < a.R) tc::tma_prefetch_2d(&tmap, 32 * int(qq % NB), int(rr));
+        if (rr < a.R) tc::tma_prefetch_2d(&tmap, EPB * int(qq % NB), int(rr));
       };
       for (long qq = 0; qq < P_PF; ++qq) prefetch(qq);
       long q = 0;
@@ -1033,7 +1060,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(P_NTH, 1)
           if (q >= P_NS) tc::mbar_wait(s.empty + sl, uint32_t((q / P_NS) - 1) & 1u);
           if (r0 < a.R) {
             tc::mbar_arrive_expect_tx(s.full + sl, 16384u);
-            tc::tma_load_2d(s.ring + sl * 4096, &tmap, 32 * b, int(r0), s.full + sl);
+            tc::tma_load_2d(s.ring + sl * 4096, &tmap, EPB * b, int(r0), s.full + sl);
           } else {
             tc::mbar_arrive(s.full + sl);                     // rows past R: nothing to load
           }
@@ -1044,7 +1071,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(P_NTH, 1)
   } else if (warp == 1) {
     // ---------------- MMA issuer (leader CTA) ----------------
     if (rank == 0) {
-      const uint32_t idsc = tc::idesc(256, uint32_t(PD), tc::FMT_F16);
+      const uint32_t idsc = tc::idesc(256, uint32_t(PD), BF ? tc::FMT_BF16 : tc::FMT_F16);
       const uint32_t w0a = tc::smem_u32(s.w0), w1a = tc::smem_u32(s.w1);
       const int nk = (K + 15) / 16;
       tc::mbar_wait(s.wfull, 0);
@@ -1063,8 +1090,10 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(P_NTH, 1)
               const uint64_t b0 = tc::sdesc_sw128(w0a + bo), b1 = tc::sdesc_sw128(w1a + bo);
               const uint32_t a0 = ah + uint32_t(kk) * 8u, a1 = a0 + 32u;
               tc::mma2_f16_ts(tmem, a0, b0, idsc, (c | kk) ? 1u : 0u);
-              tc::mma2_f16_ts(tmem, a0, b1, idsc, 1u);
-              tc::mma2_f16_ts(tmem, a1, b0, idsc, 1u);
+              if (!BF) {
+                tc::mma2_f16_ts(tmem, a0, b1, idsc, 1u);
+                tc::mma2_f16_ts(tmem, a1, b0, idsc, 1u);
+              }
             }
             tc::mma2_commit_both(s.afree + as);
             if (c == NC - 1) tc::mma2_commit_both(s.accfull);
@@ -1082,10 +1111,33 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(P_NTH, 1)
       const long r0 = row0_of(i);
       const bool live = long(row) < a.R - r0;
       float xs = 1.f;                                          // e' in [0, 1]: unscaled
-      if (EPI == EPI_NODE && live) xs = ldexpf(1.f, __ldg(a.rexp + r0 + row));
+      if (!BF && EPI == EPI_NODE && live) xs = ldexpf(1.f, __ldg(a.rexp + r0 + row));
       for (int c = 0; c < NC; ++c) {
         const long qa = long(i) * NC + c;
         const int as = int(qa % P_NA);
+        if (!AF32) {
+          // BF16 rows: one box per chunk, the row's 128 B copied into the TMEM ring as is
+          const long q = long(i) * NB + c;
+          const int sl = int(q % P_NS);
+          tc::mbar_wait(s.full + sl, uint32_t(q / P_NS) & 1u);
+          const uint8_t *box = reinterpret_cast<const uint8_t *>(s.ring + sl * 4096);
+          uint32_t w[32];
+#pragma unroll
+          for (int u = 0; u < 8; ++u) {
+            uint4 x = make_uint4(0u, 0u, 0u, 0u);
+            if (live && 64 * c + 8 * u < K)
+              x = *reinterpret_cast<const uint4 *>(box + row * 128 + ((u ^ (row & 7)) << 4));
+            w[4 * u] = x.x; w[4 * u + 1] = x.y; w[4 * u + 2] = x.z; w[4 * u + 3] = x.w;
+          }
+          tc::mbar_arrive(s.empty + sl);
+          if (qa >= P_NA) tc::mbar_wait(s.afree + as, uint32_t((qa / P_NA) - 1) & 1u);
+          tc::tmem_st32(lane_base + 256u + uint32_t(as) * 64u, w);
+          tc::tmem_st_wait();
+          tc::fence_before_sync();
+          __syncwarp();
+          if (lane == 0) tc::mbar_arrive_cluster(s.afull + as, 0);
+          continue;
+        }
         for (int kh = 0; kh < 2; ++kh) {
           const int b = 2 * c + kh;
           if (b >= NB) break;
@@ -1102,16 +1154,21 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(P_NTH, 1)
 #pragma unroll
           for (int u = 0; u < 8; ++u) {
             float4 x = v[u];
-            if (EPI == EPI_NODE) {
+            if (!BF && EPI == EPI_NODE) {
               x.x *= xs; x.y *= xs; x.z *= xs; x.w *= xs;
             }
-            split2(x.x, x.y, h[2 * u], l[2 * u]);
-            split2(x.z, x.w, h[2 * u + 1], l[2 * u + 1]);
+            if (BF) {                                          // FP32 rows rounded to BF16 (RN)
+              h[2 * u] = pack_bf16_rn(x.x, x.y);
+              h[2 * u + 1] = pack_bf16_rn(x.z, x.w);
+            } else {
+              split2(x.x, x.y, h[2 * u], l[2 * u]);
+              split2(x.z, x.w, h[2 * u + 1], l[2 * u + 1]);
+            }
           }
           if (kh == 0 && qa >= P_NA) tc::mbar_wait(s.afree + as, uint32_t((qa / P_NA) - 1) & 1u);
           const uint32_t col = 256u + uint32_t(as) * 64u + uint32_t(kh) * 16u;
           tc::tmem_st16(lane_base + col, h);
-          tc::tmem_st16(lane_base + col + 32u, l);
+          if (!BF) tc::tmem_st16(lane_base + col + 32u, l);
         }
         tc::tmem_st_wait();
         tc::fence_before_sync();
@@ -1141,7 +1198,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(P_NTH, 1)
       float aux = 0.f;
       if (EPI == EPI_EDGE && live)
         aux = __ldg(a.pin + __ldg(a.src + r0 + row)) + __ldg(a.qin + __ldg(a.dst + r0 + row));  // α
-      const int er = (EPI == EPI_NODE && live) ? __ldg(a.rexp + r0 + row) : 0;
+      const int er = (!BF && EPI == EPI_NODE && live) ? __ldg(a.rexp + r0 + row) : 0;
       tc::mbar_wait(s.accfull, uint32_t(i) & 1u);
       tc::fence_after_sync();
       uint32_t r[DQ];
@@ -1190,8 +1247,8 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(P_NTH, 1)
         for (int u = 0; u < DQ; ++u) r[u] = __float_as_uint(__uint_as_float(r[u]) * inv);
 #pragma unroll
         for (int c0 = 0; c0 < DQ; c0 += 16)
-          warp_store_chunk<PD>(wbuf, a.out, wrow0, wrows, cb + c0,
-                               *reinterpret_cast<const float (*)[16]>(r + c0), lane);
+          pair_store<BF>(wbuf, a.out, wrow0, wrows, grow, live, cb + c0,
+                         *reinterpret_cast<const float (*)[16]>(r + c0), lane);
       } else {
         float pp = 0.f, qq = 0.f;
 #pragma unroll
@@ -1216,7 +1273,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(P_NTH, 1)
               for (int t = 0; t < 4; ++t) o[u + t] = fast_rcp(1.f + ex2(__uint_as_float(r[c0 + u + t]) * cexp));
             }
           }
-          warp_store_chunk<PD>(wbuf, a.out, wrow0, wrows, cb + c0, o, lane);
+          pair_store<BF>(wbuf, a.out, wrow0, wrows, grow, live, cb + c0, o, lane);
         }
         if (EPI == EPI_NODE) {
           s.xch[cq * 128 + row] = pp;
@@ -2241,21 +2298,44 @@ static int launch_rowgemm(const occu_ctx *ctx, const RowGemmArgs &ra, const char
   return 1;
 }
 
-// d = 256: CTA-pair row-GEMM (rowgemm_pair_kernel), grid = 2 x clusters
-template <int EPI>
+// BF16 rows [R][K]: boxes of 128 rows x 64 bf16 (128 B), 128-byte swizzle, OOB zero
+static bool encode_rows_map_bf16_128(CUtensorMap *m, const void *A, long R, int K) {
+  static PFN_encodeTiled fn = nullptr;
+  if (!fn) {
+    void *p = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) != cudaSuccess ||
+        q != cudaDriverEntryPointSuccess || !p)
+      return false;
+    fn = reinterpret_cast<PFN_encodeTiled>(p);
+  }
+  const cuuint64_t dims[2] = {cuuint64_t(K), cuuint64_t(R)};
+  const cuuint64_t strides[1] = {cuuint64_t(K) * 2};
+  const cuuint32_t box[2] = {64, 128};
+  const cuuint32_t estr[2] = {1, 1};
+  return fn(m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void *>(A), dims, strides, box, estr,
+            CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+            CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
+// d = 256: CTA-pair row-GEMM (rowgemm_pair_kernel), grid = 2 x clusters.  FP32 mode (BF =
+// false): FP32 rows, per-row scale exponents for node inputs first (row_exp_kernel).
+template <int EPI, bool BF, bool AF32>
 static int launch_rowgemm_pair(const occu_ctx *ctx, RowGemmArgs ra, const char *name,
                                cudaStream_t st) {
+  static_assert(BF || AF32, "OCCU_FP32 rows are FP32");
   if (ra.R <= 0) return 0;
-  if (ra.K > 256) return -int(cudaErrorInvalidValue);
-  const size_t smem = pair_smem_bytes(ra.K);
-  set_smem(rowgemm_pair_kernel<EPI>, smem);
+  if (ra.K > 256 || (!AF32 && ra.K % 64)) return -int(cudaErrorInvalidValue);
+  const size_t smem = pair_smem_bytes(ra.K, BF ? 1 : 2);
+  set_smem(rowgemm_pair_kernel<EPI, BF, AF32>, smem);
   const int tiles = (ra.R + 2 * TM - 1) / (2 * TM);
   const int clusters = std::max(1, std::min(tiles, ctx->num_sms / 2));
   CUtensorMap tmap;
-  if (!encode_rows_map(&tmap, ra.A, ra.R, ra.K)) return -int(cudaErrorInvalidValue);
+  if (!(AF32 ? encode_rows_map(&tmap, ra.A, ra.R, ra.K) : encode_rows_map_bf16_128(&tmap, ra.A, ra.R, ra.K)))
+    return -int(cudaErrorInvalidValue);
   int n = 0;
   OCCU_PROF_BEGIN(ctx, name, st);
-  if (EPI == EPI_NODE) {          // the rows' scale exponents first
+  if (!BF && EPI == EPI_NODE) {          // the rows' scale exponents first
     if (const_cast<occu_ctx *>(ctx)->ws.rowexp.ensure(size_t(ra.R) * 4) != cudaSuccess)
       return -int(cudaErrorMemoryAllocation);
     int *rexp = ctx->ws.rowexp.as<int>();
@@ -2264,7 +2344,7 @@ static int launch_rowgemm_pair(const occu_ctx *ctx, RowGemmArgs ra, const char *
     launch_pdl(ctx->pdl & 1, row_exp_kernel, g, 256, 0, st, ra.A, ra.R, ra.K, rexp);
     ++n;
   }
-  launch_pdl(ctx->pdl & 1, rowgemm_pair_kernel<EPI>, 2 * clusters, P_NTH, smem, st, tmap, ra);
+  launch_pdl(ctx->pdl & 1, rowgemm_pair_kernel<EPI, BF, AF32>, 2 * clusters, P_NTH, smem, st, tmap, ra);
   OCCU_PROF_END(ctx);
   TC_CHECK();
   return n + 1;
@@ -2283,7 +2363,7 @@ static int tc_forward_layer_pair(const occu_ctx *ctx, const DevCsr &csr, int lay
   ra.wimg = tc_wimg(ctx, 0, layer); ra.wfexp = tc_wfexp(ctx, 0, layer);
   ra.a_s = a.a_s; ra.a_d = a.a_d; ra.p = a.p; ra.q = a.q;
   ra.rev = ctx->l2_order;
-  if ((r = launch_rowgemm_pair<EPI_NODE>(ctx, ra, "node_tc", st)) < 0) return r;
+  if ((r = launch_rowgemm_pair<EPI_NODE, false, true>(ctx, ra, "node_tc", st)) < 0) return r;
   n += r;
   if (csr.E > 0) {
     if (a.Ke <= 16) {
@@ -2304,7 +2384,7 @@ static int tc_forward_layer_pair(const occu_ctx *ctx, const DevCsr &csr, int lay
       re.A = a.e_in; re.K = a.Ke; re.R = csr.E; re.W = a.W_e; re.out = a.e_out;
       re.wimg = tc_wimg(ctx, 1, layer); re.wfexp = tc_wfexp(ctx, 1, layer);
       re.pin = a.p; re.qin = a.q; re.src = csr.in_src; re.dst = csr.in_dst;
-      if ((r = launch_rowgemm_pair<EPI_EDGE>(ctx, re, "edge_tc", st)) < 0) return r;
+      if ((r = launch_rowgemm_pair<EPI_EDGE, false, true>(ctx, re, "edge_tc", st)) < 0) return r;
       n += r;
     }
     RowGemmArgs rg{};
@@ -2312,7 +2392,7 @@ static int tc_forward_layer_pair(const occu_ctx *ctx, const DevCsr &csr, int lay
     rg.A = a.e_out; rg.K = D; rg.R = csr.E; rg.W = a.W_m; rg.out = a.g;
     rg.wimg = tc_wimg(ctx, 2, layer); rg.wfexp = tc_wfexp(ctx, 2, layer);
     rg.rev = ctx->l2_order;
-    if ((r = launch_rowgemm_pair<EPI_GATE>(ctx, rg, "gate_tc", st)) < 0) return r;
+    if ((r = launch_rowgemm_pair<EPI_GATE, false, true>(ctx, rg, "gate_tc", st)) < 0) return r;
     n += r;
   }
   if ((r = launch_gather_segsum(ctx, csr, a.g, a.hbar, a.h_out, a.rpart, st)) < 0) return r;
@@ -2566,6 +2646,29 @@ int launch_bwd_edge_tc(const occu_ctx *ctx, const DevCsr &csr, int layer, const 
   if (csr.E <= 0) return 0;
   return ctx->cfg.d == 64 ? bwd_edge_impl<64>(ctx, csr, layer, e_in, Ke, e, de, p, q, DZ, dal, st)
                           : bwd_edge_impl<128>(ctx, csr, layer, e_in, Ke, e, de, p, q, DZ, dal, st);
+}
+
+// OCCU_BF16 at d = 256 (kernels_bf16.cu): the pair row-GEMM of one forward step.
+// epi: 0 node (A = layer-1 FP32 features if af32, else BF16 h), 1 edge, 2 gate; out BF16.
+int launch_pair_bf16(const occu_ctx *ctx, int epi, bool af32, const void *A, int K, int R, int layer,
+                     void *out, const float *a_s, const float *a_d, float *p, float *q,
+                     const int32_t *src, const int32_t *dst, const char *name, cudaStream_t st) {
+  RowGemmArgs ra{};
+  ra.slope = ctx->cfg.slope;
+  ra.A = static_cast<const float *>(A); ra.K = K; ra.R = R;
+  ra.out = static_cast<float *>(out);
+  ra.wimg = tc_wimg(ctx, epi, layer); ra.wfexp = tc_wfexp(ctx, epi, layer);
+  ra.a_s = a_s; ra.a_d = a_d; ra.p = p; ra.q = q;
+  ra.pin = p; ra.qin = q; ra.src = src; ra.dst = dst;
+  ra.rev = epi == 1 ? 0 : ctx->l2_order;
+  switch (epi * 2 + (af32 ? 1 : 0)) {
+    case 0: return launch_rowgemm_pair<EPI_NODE, true, false>(ctx, ra, name, st);
+    case 1: return launch_rowgemm_pair<EPI_NODE, true, true>(ctx, ra, name, st);
+    case 2: return launch_rowgemm_pair<EPI_EDGE, true, false>(ctx, ra, name, st);
+    case 3: return launch_rowgemm_pair<EPI_EDGE, true, true>(ctx, ra, name, st);
+    case 4: return launch_rowgemm_pair<EPI_GATE, true, false>(ctx, ra, name, st);
+    default: return -int(cudaErrorInvalidValue);
+  }
 }
 
 int launch_forward_layer_tc(const occu_ctx *ctx, const DevCsr &csr, int layer, const FwdLayerArgs &a,

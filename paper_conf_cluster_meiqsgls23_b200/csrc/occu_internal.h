@@ -239,6 +239,9 @@ int launch_gather_segsoftmax_bf16(const occu_ctx *ctx, const DevCsr &csr, void *
 int launch_gather_segsum_bf16(const occu_ctx *ctx, const DevCsr &csr, const void *g,
                               const void *hbar, void *h_out, float *rpart, cudaStream_t st);
 // OCCU_BF16 forward layer (kernels_bf16.cu); FwdLayerArgs pointers to h̄, e', g, h hold BF16.
+int launch_pair_bf16(const occu_ctx *ctx, int epi, bool af32, const void *A, int K, int R, int layer,
+                     void *out, const float *a_s, const float *a_d, float *p, float *q,
+                     const int32_t *src, const int32_t *dst, const char *name, cudaStream_t st);
 int launch_forward_layer_bf16(const occu_ctx *ctx, const DevCsr &csr, int layer,
                               const FwdLayerArgs &a, cudaStream_t st);
 int launch_permute_rows(const occu_ctx *ctx, const float *src, const int32_t *idx, int rows,

@@ -153,10 +153,10 @@ occu_status validate_cfg(const occu_config *c) {
   if (c->L < 1 || c->L > 16) return fail(nullptr, OCCU_EINVAL, "L must be in [1, 16]");
   if (c->d != 64 && c->d != 128 && c->d != 256)
     return fail(nullptr, OCCU_EINVAL, "this build supports d in {64, 128, 256}");
-  if (c->d == 256 && (c->prec != OCCU_FP32 || c->msg != OCCU_MSG_CHANNEL_SOFTMAX ||
-                      c->readout != OCCU_READOUT_MEAN || c->graphormer != 0))
+  if (c->d == 256 && (c->msg != OCCU_MSG_CHANNEL_SOFTMAX || c->readout != OCCU_READOUT_MEAN ||
+                      c->graphormer != 0 || (c->prec == OCCU_BF16 && c->F_e > 16)))
     return fail(nullptr, OCCU_EINVAL,
-                "d = 256 (CTA-pair tensor-core path) supports OCCU_FP32, reading A, the mean readout and no Graphormer layers");
+                "d = 256 (CTA-pair tensor-core path) supports reading A, the mean readout, no Graphormer layers (OCCU_BF16: F_e <= 16)");
   if (c->F_n < 4 || c->F_n % 4 || c->F_n > 256 || c->F_e < 4 || c->F_e % 4 || c->F_e > 256)
     return fail(nullptr, OCCU_EINVAL, "F_n, F_e must be multiples of 4 in [4, 256]");
   if (c->d_h < 1 || c->d_h > 1024) return fail(nullptr, OCCU_EINVAL, "d_h must be in [1, 1024]");

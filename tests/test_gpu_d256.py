@@ -144,3 +144,44 @@ def test_training_at_d256_fails_loudly():
     csr = occu.pack(b.graphs)
     with pytest.raises(Exception):
         m.train_step(csr, b.node_feat, b.edge_feat, b.targets, 1e-4)
+
+
+# ---- OCCU_BF16 at d = 256 (R48): the pair kernels with BF16 operands and stored activations,
+# checked as tests/test_gpu_bf16.py checks d <= 128: every intermediate vs the oracle's
+# BF16-mode forward (same roundings, float64) at 3e-3, ŷ vs the float64 oracle at 1e-2
+# (rel-L2 and per graph with the 0.1 floor, R25)
+TOL_BF = 1e-2
+TOL_EMU = 3e-3
+
+
+@pytest.mark.parametrize("L,aggr,seed,unit", [(1, 0, 31, True), (2, 1, 32, True), (3, 0, 33, False)])
+def test_bf16_random_batches_all_intermediates(L, aggr, seed, unit):
+    c = occu.config(L=L, F_n=80, F_e=4, d=256, aggr=aggr, prec=occu.BF16)
+    b = configs.random_dag_batch(40, 760 + seed, max_nodes=60, hub=True)
+    flat = weights.init_flat(wcfg(c), seed)
+    if unit:
+        flat = weights.unit_scale(wcfg(c), flat)
+    m, y, ref, pk = run_both(c, b, flat)
+    emu = oracle.forward_bf16(oracle.unflatten(ocfg(c), flat.astype(np.float64)), ocfg(c), pk,
+                              b.node_feat, b.edge_feat)
+    N, E, B = pk["num_nodes"], pk["num_edges"], pk["num_graphs"]
+    for i in range(L):
+        lay = emu["layers"][i]
+        for name, t, shape in (("hbar", occu.T_HBAR, (N, 256)), ("p", occu.T_P, (N,)), ("q", occu.T_Q, (N,)),
+                               ("e", occu.T_E, (E, 256)), ("h", occu.T_H, (N, 256))):
+            assert rel(m.get_tensor(t, i, shape), lay[name]) <= TOL_EMU, (name, i)
+    assert rel(m.get_tensor(occu.T_R, 0, (B, 256)), emu["r"]) <= TOL_EMU
+    assert rel(y, emu["yhat"]) <= TOL_EMU
+    yr = ref["yhat"]
+    assert rel(y, yr) <= TOL_BF
+    assert np.all(np.abs(y - yr) <= TOL_BF * np.maximum(np.abs(yr), 0.1)), np.abs(y - yr).max()
+
+
+def test_bf16_paper_encoder_shape_cfg2_graphs():
+    c = occu.config(L=1, F_n=80, F_e=4, d=256, prec=occu.BF16)
+    b = configs.cfg2(48)
+    flat = weights.unit_scale(wcfg(c), weights.init_flat(wcfg(c), 22))
+    m, y, ref, pk = run_both(c, b, flat, keep=False)
+    yr = ref["yhat"]
+    assert rel(y, yr) <= TOL_BF
+    assert np.all(np.abs(y - yr) <= TOL_BF * np.maximum(np.abs(yr), 0.1)), np.abs(y - yr).max()
