@@ -45,7 +45,8 @@ def test_bench_default_line_contract():
     # every secondary section ran (a failed section is reported on stderr and has no entry)
     assert "FAILED" not in out.stderr, out.stderr[-3000:]
     for k in ("cfg3_train_bf16", "cfg2_infer_f32", "cfg2_infer_bf16", "cfg1_latency_us",
-              "cfg4_epoch_bf16", "cfg5_sweep_1M_bf16"):
+              "cfg4_epoch_bf16", "cfg5_sweep_1M_bf16", "cfg2_paper_f32", "cfg2_paper_bf16",
+              "cfg2_paper_stack_train_f32"):
         assert k in j["secondary"], k
     assert j["aggregation"]["kernel"] == "gather_segsum"
 
