@@ -1052,12 +1052,15 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(P_NTH, 1)
       };
       for (long qq = 0; qq < P_PF; ++qq) prefetch(qq);
       long q = 0;
+      TT_DECL
       for (int i = 0; i < my; ++i) {
         const long r0 = row0_of(i);
         for (int b = 0; b < NB; ++b, ++q) {
           const int sl = int(q % P_NS);
           prefetch(q + P_PF);
+          TT_WAIT_BEGIN
           if (q >= P_NS) tc::mbar_wait(s.empty + sl, uint32_t((q / P_NS) - 1) & 1u);
+          TT_WAIT_END
           if (r0 < a.R) {
             tc::mbar_arrive_expect_tx(s.full + sl, 16384u);
             tc::tma_load_2d(s.ring + sl * 4096, &tmap, EPB * b, int(r0), s.full + sl);
@@ -1066,6 +1069,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(P_NTH, 1)
           }
         }
       }
+      if (EPI == EPI_GATE) TT_FLUSH(0);
     }
     __syncwarp();
   } else if (warp == 1) {
@@ -1076,12 +1080,17 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(P_NTH, 1)
       const int nk = (K + 15) / 16;
       tc::mbar_wait(s.wfull, 0);
       tc::mbar_wait_cluster(s.wpeer, 0);
+      TT_DECL
       for (int i = 0; i < my; ++i) {
+        TT_WAIT_BEGIN
         if (i >= 1) tc::mbar_wait_cluster(s.accfree, uint32_t(i - 1) & 1u);
+        TT_WAIT_END
         for (int c = 0; c < NC; ++c) {
           const long qa = long(i) * NC + c;
           const int as = int(qa % P_NA);
+          TT_WAIT_BEGIN
           tc::mbar_wait_cluster(s.afull + as, uint32_t(qa / P_NA) & 1u);
+          TT_WAIT_END
           tc::fence_after_sync();
           if (lane == 0) {
             const uint32_t ah = tmem + 256u + uint32_t(as) * 64u;
@@ -1101,12 +1110,14 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(P_NTH, 1)
           __syncwarp();
         }
       }
+      if (EPI == EPI_GATE) TT_FLUSH(1);
     }
   } else if (warp < P_EPI0) {
     // ---------------- converters: thread = row -> TMEM A ring ----------------
     const int qd = warp & 3;
     const int row = qd * 32 + lane;
     const uint32_t lane_base = tmem + (uint32_t(qd * 32) << 16);
+    TT_DECL
     for (int i = 0; i < my; ++i) {
       const long r0 = row0_of(i);
       const bool live = long(row) < a.R - r0;
@@ -1143,7 +1154,9 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(P_NTH, 1)
           if (b >= NB) break;
           const long q = long(i) * NB + b;
           const int sl = int(q % P_NS);
+          TT_WAIT_BEGIN
           tc::mbar_wait(s.full + sl, uint32_t(q / P_NS) & 1u);
+          TT_WAIT_END
           const float *box = s.ring + sl * 4096;
           float4 v[8];
 #pragma unroll
@@ -1165,7 +1178,9 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(P_NTH, 1)
               split2(x.z, x.w, h[2 * u + 1], l[2 * u + 1]);
             }
           }
+          TT_WAIT_BEGIN
           if (kh == 0 && qa >= P_NA) tc::mbar_wait(s.afree + as, uint32_t((qa / P_NA) - 1) & 1u);
+          TT_WAIT_END
           const uint32_t col = 256u + uint32_t(as) * 64u + uint32_t(kh) * 16u;
           tc::tmem_st16(lane_base + col, h);
           if (!BF) tc::tmem_st16(lane_base + col + 32u, l);
@@ -1176,6 +1191,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(P_NTH, 1)
         if (lane == 0) tc::mbar_arrive_cluster(s.afull + as, 0);
       }
     }
+    if (EPI == EPI_GATE) TT_FLUSH(2 + (warp - 2));
     // the last chunks' MMAs (and their commits to this CTA) must land before teardown
     for (long qa = max(0L, long(my) * NC - P_NA); qa < long(my) * NC; ++qa)
       tc::mbar_wait(s.afree + int(qa % P_NA), uint32_t(qa / P_NA) & 1u);
@@ -1191,6 +1207,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(P_NTH, 1)
     float *wbuf = s.xbuf + wi * (16 * 20);
     constexpr int DQ = PD / 4;
     const int cb = cq * DQ;
+    TT_DECL
     for (int i = 0; i < my; ++i) {
       const long r0 = row0_of(i);
       const int nrows = int(max(0L, min(long(TM), a.R - r0)));
@@ -1199,7 +1216,9 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(P_NTH, 1)
       if (EPI == EPI_EDGE && live)
         aux = __ldg(a.pin + __ldg(a.src + r0 + row)) + __ldg(a.qin + __ldg(a.dst + r0 + row));  // α
       const int er = (!BF && EPI == EPI_NODE && live) ? __ldg(a.rexp + r0 + row) : 0;
+      TT_WAIT_BEGIN
       tc::mbar_wait(s.accfull, uint32_t(i) & 1u);
+      TT_WAIT_END
       tc::fence_after_sync();
       uint32_t r[DQ];
       {
@@ -1287,6 +1306,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(P_NTH, 1)
       }
       epi_bar_pair();          // the exchange area is reused by the next tile
     }
+    if (EPI == EPI_GATE) TT_FLUSH(6 + wi);
   }
   tc::fence_before_sync();
   __syncthreads();
