@@ -32,6 +32,11 @@ struct SmallArgs {
 };
 
 __device__ __forceinline__ float lrelu_s(float x, float s) { return x > 0.f ? x : s * x; }
+__device__ __forceinline__ float ex2_fast(float x) {
+  float r;
+  asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(r) : "f"(x));
+  return r;
+}
 
 #ifdef OCCU_SMALL_TIMING
 __device__ unsigned long long g_small_ts[64];
@@ -190,7 +195,7 @@ __global__ void __launch_bounds__(ST, 1) small_forward_kernel(const SmallArgs a)
     for (int i = t; i < E * d; i += ST) {
       const int k = i / d;
       const float al = pq[isrc[k]] + pq[SNMAX + idst[k]];
-      Eout[i] = __frcp_rn(1.f + exp2f(-al * Ev[i] * 1.4426950408889634f));
+      Eout[i] = __fdividef(1.f, 1.f + ex2_fast(-al * Ev[i] * 1.4426950408889634f));
     }
     // a4: logits W_m e', softmax over the d channels (warp per edge)
     if (l + 1 < a.L) cpa_wait<1>(); else cpa_wait<0>();
@@ -205,7 +210,7 @@ __global__ void __launch_bounds__(ST, 1) small_forward_kernel(const SmallArgs a)
       for (int o = 16; o > 0; o >>= 1) m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, o));
       float s = 0.f;
       for (int c = lane; c < d; c += 32) {
-        const float x = exp2f((Ev[k * d + c] - m) * 1.4426950408889634f);
+        const float x = ex2_fast((Ev[k * d + c] - m) * 1.4426950408889634f);
         Ev[k * d + c] = x;
         s += x;
       }
