@@ -185,3 +185,31 @@ def test_bf16_paper_encoder_shape_cfg2_graphs():
     yr = ref["yhat"]
     assert rel(y, yr) <= TOL_BF
     assert np.all(np.abs(y - yr) <= TOL_BF * np.maximum(np.abs(yr), 0.1)), np.abs(y - yr).max()
+
+
+def test_d256_deterministic_and_batching_invariant():
+    """Reruns are bitwise equal (fixed-order sums, no atomics in the pair kernels); a graph
+    predicted alone agrees with its prediction inside a batch at the FP32 tolerance."""
+    c = mk(2)
+    b = configs.random_dag_batch(30, 951, max_nodes=50, hub=True)
+    flat = weights.unit_scale(wcfg(c), weights.init_flat(wcfg(c), 13))
+    m = occu.Model(c)
+    m.set_params(flat)
+    csr = occu.pack(b.graphs)
+    y1 = m.predict(csr, b.node_feat, b.edge_feat)
+    y2 = m.predict(csr, b.node_feat, b.edge_feat)
+    assert np.array_equal(y1, y2)
+    n0 = b.graphs[0][0]
+    e0 = len(b.graphs[0][1])
+    y0 = m.predict(occu.pack(b.graphs[:1]), b.node_feat[:n0], b.edge_feat[:e0])
+    assert abs(float(y0[0]) - float(y1[0])) <= TOL * max(abs(float(y1[0])), 1e-2)
+
+
+@pytest.mark.parametrize("kw", [dict(msg=1), dict(readout=1, k=4, heads=4), dict(graphormer=1, heads=4),
+                                dict(prec=1, F_e=64)])
+def test_d256_unsupported_modes_fail_loudly(kw):
+    """Modes outside R48's scope are rejected at creation (OCCU_EINVAL), not run on another path."""
+    base = dict(L=1, F_n=80, F_e=4, d=256)
+    base.update(kw)
+    with pytest.raises(Exception):
+        occu.Model(occu.config(**base))
