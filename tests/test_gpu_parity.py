@@ -424,6 +424,34 @@ def test_predict_async_pipeline_matches_predict():
                         torch.from_numpy(b.edge_feat).to(dev), torch.empty(b.num_graphs, device=dev))
 
 
+def test_predict_async_keeps_temporary_outputs_alive():
+    """The binding holds every output tensor passed to predict_async until wait(): with the
+    caller's references dropped and a garbage collection in between, all outputs are still
+    alive and each receives its batch's predictions (the D2H of call k may still
+    be in flight when call k+1 returns)."""
+    import gc
+    import weakref
+    import torch
+    c = mk(2, 64)
+    m = occu.Model(c)
+    m.init_weights(7)
+    batches = [configs.random_dag_batch(20 + 3 * k, 1300 + k, max_nodes=40) for k in range(3)]
+    want = [m.predict(occu.pack(b.graphs), b.node_feat, b.edge_feat) for b in batches]
+    ins = [(torch.from_numpy(b.node_feat).pin_memory(), torch.from_numpy(b.edge_feat).pin_memory()) for b in batches]
+    refs = []
+    for b, (nf, ef) in zip(batches, ins):
+        out = torch.full((b.num_graphs,), float("nan")).pin_memory()
+        refs.append(weakref.ref(out))
+        m.predict_async(occu.pack(b.graphs), nf, ef, out)
+        del out
+    gc.collect()
+    outs = [r() for r in refs]             # alive only through the binding's references
+    assert all(o is not None for o in outs)
+    m.wait()
+    for o, w in zip(outs, want):
+        assert np.array_equal(o.numpy(), w)
+
+
 def test_cfg5_mixture_launch_sampled_graphs():
     """BASELINE CFG5's launch unit: 1,024 graphs of the 20-family mixture (1.4 M nodes) on
     device buffers, FP32 and OCCU_BF16; one sampled graph of every family present checked
