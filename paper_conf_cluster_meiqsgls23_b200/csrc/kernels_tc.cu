@@ -917,12 +917,14 @@ struct PairSmem {
   float *avec;                        // [2][256] a_s, a_d (NODE)
   float *xch;                         // [2 values][4 quarters][128 rows]
   float *xbuf;                        // 16 epilogue warps x 16 x 20 floats
+  uint64_t *eready;                   // [4] row exponents of tile i in erow (local row max)
+  int *erow;                          // [4][128]
 };
 
 // nimg: 2 fp16x2 images (OCCU_FP32) or 1 BF16 image (OCCU_BF16)
 __host__ __device__ inline size_t pair_smem_bytes(int K, int nimg) {
   const size_t img = size_t(kpad_of(K)) * 128 * 2;
-  return 1024 + nimg * img + size_t(P_NS) * 16384 + 256 + 2048 + 4096 + 16 * 16 * 20 * 4;
+  return 1024 + nimg * img + size_t(P_NS) * 16384 + 256 + 2048 + 4096 + 16 * 16 * 20 * 4 + 4 * 128 * 4;
 }
 
 __device__ __forceinline__ PairSmem carve_pair(uint8_t *raw, int K, int nimg) {
@@ -943,10 +945,12 @@ __device__ __forceinline__ PairSmem carve_pair(uint8_t *raw, int K, int nimg) {
   s.accfree = s.accfull + 1;
   s.wfull = s.accfull + 2;
   s.wpeer = s.accfull + 3;
+  s.eready = s.accfull + 4;           // 4
   s.tmem_slot = reinterpret_cast<uint32_t *>(misc + 224);
   s.avec = reinterpret_cast<float *>(misc + 256);
   s.xch = reinterpret_cast<float *>(misc + 256 + 2048);
   s.xbuf = reinterpret_cast<float *>(misc + 256 + 2048 + 4096);
+  s.erow = reinterpret_cast<int *>(misc + 256 + 2048 + 4096 + 16 * 16 * 20 * 4);
   return s;
 }
 
@@ -1001,6 +1005,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(P_NTH, 1)
     tc::mbar_init(s.accfree, 32);       // 16 epilogue warps x 2 CTAs (leader's copy used)
     tc::mbar_init(s.wfull, 1);
     tc::mbar_init(s.wpeer, 1);
+    for (int j = 0; j < 4; ++j) tc::mbar_init(s.eready + j, 128);
     tc::fence_mbar_init();
   }
   if (warp == 1) tc::tmem_alloc2<TMEM_COLS>(s.tmem_slot);
@@ -1122,7 +1127,32 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(P_NTH, 1)
       const long r0 = row0_of(i);
       const bool live = long(row) < a.R - r0;
       float xs = 1.f;                                          // e' in [0, 1]: unscaled
-      if (!BF && EPI == EPI_NODE && live) xs = ldexpf(1.f, __ldg(a.rexp + r0 + row));
+      if (!BF && EPI == EPI_NODE) {
+        if (a.rexp) {                                          // exponents from row_exp_kernel
+          if (live) xs = ldexpf(1.f, __ldg(a.rexp + r0 + row));
+        } else {
+          // K <= 128: the tile's NB <= P_NS boxes are all in the ring at once; the row max
+          // is taken over them before any box is released (no row_exp_kernel pass)
+          float mx = 0.f;
+          for (int b = 0; b < NB; ++b) {
+            const long q = long(i) * NB + b;
+            const int sl = int(q % P_NS);
+            tc::mbar_wait(s.full + sl, uint32_t(q / P_NS) & 1u);
+            const float *box = s.ring + sl * 4096;
+            if (live)
+#pragma unroll
+              for (int u = 0; u < 8; ++u)
+                if (32 * b + 4 * u < K) {
+                  const float4 v = slot_ld4(box, row, 4 * u);
+                  mx = fmaxf(mx, fmaxf(fmaxf(fabsf(v.x), fabsf(v.y)), fmaxf(fabsf(v.z), fabsf(v.w))));
+                }
+          }
+          const int er = scale_exp(mx);
+          xs = ldexpf(1.f, er);
+          s.erow[(i & 3) * 128 + row] = er;
+          tc::mbar_arrive(s.eready + (i & 3));
+        }
+      }
       for (int c = 0; c < NC; ++c) {
         const long qa = long(i) * NC + c;
         const int as = int(qa % P_NA);
@@ -1215,7 +1245,15 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(P_NTH, 1)
       float aux = 0.f;
       if (EPI == EPI_EDGE && live)
         aux = __ldg(a.pin + __ldg(a.src + r0 + row)) + __ldg(a.qin + __ldg(a.dst + r0 + row));  // α
-      const int er = (!BF && EPI == EPI_NODE && live) ? __ldg(a.rexp + r0 + row) : 0;
+      int er = 0;
+      if (!BF && EPI == EPI_NODE) {
+        if (a.rexp) {
+          if (live) er = __ldg(a.rexp + r0 + row);
+        } else {
+          tc::mbar_wait(s.eready + (i & 3), uint32_t(i >> 2) & 1u);
+          er = s.erow[(i & 3) * 128 + row];
+        }
+      }
       TT_WAIT_BEGIN
       tc::mbar_wait(s.accfull, uint32_t(i) & 1u);
       TT_WAIT_END
@@ -2355,7 +2393,8 @@ static int launch_rowgemm_pair(const occu_ctx *ctx, RowGemmArgs ra, const char *
     return -int(cudaErrorInvalidValue);
   int n = 0;
   OCCU_PROF_BEGIN(ctx, name, st);
-  if (!BF && EPI == EPI_NODE) {          // the rows' scale exponents first
+  ra.rexp = nullptr;
+  if (!BF && EPI == EPI_NODE && (ra.K + 31) / 32 > P_NS) {   // K > 128: the rows' scale exponents first
     if (const_cast<occu_ctx *>(ctx)->ws.rowexp.ensure(size_t(ra.R) * 4) != cudaSuccess)
       return -int(cudaErrorMemoryAllocation);
     int *rexp = ctx->ws.rowexp.as<int>();
