@@ -23,7 +23,7 @@ OUT = os.environ.get("PROFILES_OUT", os.path.join(ROOT, "profiles"))
 
 def kname(full):
     import re
-    m = re.search(r"rowgemm_pair_kernel<(?:\(int\))?(\d+)>", full)
+    m = re.search(r"rowgemm_pair_kernel<(?:\(int\))?(\d+)[,>]", full)
     if m:
         return ["node_tc", "edge_tc", "gate_tc"][int(m.group(1))]
     m = re.search(r"rowgemm(?:_bf16)?_kernel<(?:\(int\))?(\d+), (?:\(int\))?(\d+)", full)
