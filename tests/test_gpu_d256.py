@@ -213,3 +213,17 @@ def test_d256_unsupported_modes_fail_loudly(kw):
     base.update(kw)
     with pytest.raises(Exception):
         occu.Model(occu.config(**base))
+
+
+@pytest.mark.parametrize("F_n", [200, 256])
+def test_wide_node_features(F_n):
+    """F_n > 128: the layer-1 node transform takes its row scales from row_exp_kernel and
+    (F_n = 200) ends in a partial 64-wide K chunk with a missing last box."""
+    c = mk(1, F_n=F_n)
+    b = configs.random_dag_batch(20, 980 + F_n, max_nodes=50, hub=True)
+    rng = np.random.default_rng(F_n)
+    nf = (rng.standard_normal((b.num_nodes, F_n)) * np.exp(rng.uniform(-3, 3, (b.num_nodes, 1)))).astype(np.float32)
+    b = configs.Batch(b.graphs, nf, b.edge_feat, b.targets, b.families)
+    flat = weights.unit_scale(wcfg(c), weights.init_flat(wcfg(c), 14))
+    m, y, ref, pk = run_both(c, b, flat)
+    compare_all(m, c, y, ref, pk)
