@@ -1050,14 +1050,26 @@ struct DecPoolBwdArgs {
 // nearly coincide across a graph no longer cancel at the size of Z itself.
 template <int D>
 __global__ void __launch_bounds__(DT) dec_pool_bwd_kernel(const DecPoolBwdArgs a, int mode) {
-  __shared__ __align__(16) float Zc[CH][D];
+  // the folded key map (prep: [c][kh] + the bias row) and the graph's u vectors are staged in
+  // shared memory once per CTA (row strides padded to D + 1: conflict-free column walks);
+  // every sum keeps its order (the same bits as reading them from global memory)
+  __shared__ float Zc[CH][D + 1];
   __shared__ float al[CH][KHMAX], ds[CH][KHMAX];
   __shared__ float Dsum[KHMAX];
-  __shared__ __align__(16) float Zr[D];
+  __shared__ float Zr[D];
+  __shared__ float Ps[D * KHMAX + KHMAX];      // prep [c][kh], then the bias row [kh]
+  __shared__ float PsT[KHMAX][D + 1];           // prep transposed [kh][c]
+  __shared__ float Us[KHMAX][D + 1];            // u of graph g [kh][c]
   const int KH = a.k * a.heads, t = threadIdx.x, g = blockIdx.x, sp = blockIdx.y;
   const long g0 = a.node_off[g], len = a.node_off[g + 1] - g0;
   const long u0 = g0 + len * sp / SPLIT, u1 = g0 + len * (sp + 1) / SPLIT;
   for (int c = t; c < D; c += DT) Zr[c] = __ldg(a.Z + g0 * D + c);
+  for (int i = t; i < D * KHMAX + KHMAX; i += DT) {
+    const float v = a.prep[i];
+    Ps[i] = v;
+    if (i < D * KHMAX) PsT[i % KHMAX][i / KHMAX] = v;
+  }
+  for (int i = t; i < KHMAX * D; i += DT) Us[i / D][i % D] = __ldg(a.u + long(g) * KHMAX * D + i);
   if (mode == 1 && t < KH) {
     float s = 0.f;
     for (int q = 0; q < SPLIT; ++q) s += a.dsum_part[(long(g) * SPLIT + q) * KHMAX + t];
@@ -1080,11 +1092,11 @@ __global__ void __launch_bounds__(DT) dec_pool_bwd_kernel(const DecPoolBwdArgs a
     __syncthreads();
     for (int o = t; o < rows * KH; o += DT) {       // α and ∂α − ∂α_r of (row, kh)
       const int r = o / KH, kh = o % KH;
-      float s = a.prep[D * KHMAX + kh], da = 0.f;
-      const float *uk = a.u + (long(g) * KHMAX + kh) * D;
+      float s = Ps[D * KHMAX + kh], da = 0.f;
+#pragma unroll 8
       for (int c = 0; c < D; ++c) {
-        s = fmaf(Zc[r][c], a.prep[c * KHMAX + kh], s);
-        da = fmaf(Zc[r][c] - Zr[c], __ldg(uk + c), da);
+        s = fmaf(Zc[r][c], Ps[c * KHMAX + kh], s);
+        da = fmaf(Zc[r][c] - Zr[c], Us[kh][c], da);
       }
       const float M = a.pstat[(long(g) * KHMAX + kh) * 2], l = a.pstat[(long(g) * KHMAX + kh) * 2 + 1];
       const float alpha = ex2((s - M) * L2E) / l;
@@ -1100,7 +1112,7 @@ __global__ void __launch_bounds__(DT) dec_pool_bwd_kernel(const DecPoolBwdArgs a
         const int r = o / D, c = o % D;
         float z = 0.f;
         for (int kh = 0; kh < KH; ++kh)
-          z = fmaf(al[r][kh], __ldg(a.u + (long(g) * KHMAX + kh) * D + c), fmaf(ds[r][kh], a.prep[c * KHMAX + kh], z));
+          z = fmaf(al[r][kh], Us[kh][c], fmaf(ds[r][kh], PsT[kh][c], z));
         a.dZ[(n0 + r) * D + c] = z;
       }
 #pragma unroll
@@ -1127,6 +1139,30 @@ __global__ void __launch_bounds__(DT) dec_pool_bwd_kernel(const DecPoolBwdArgs a
   }
 }
 
+// Merge of the pool-backward partials over graphs and ranges, thread per output (kh, c):
+// Σ_g Σ_q in float64, g ascending then q ascending (the order the seeds' CTA used to walk
+// alone); consecutive threads read consecutive columns of each partial row.
+__global__ void __launch_bounds__(256) dec_gpart_reduce_kernel(const float *__restrict__ gpart, int B, int KH,
+                                                               int W, float *__restrict__ gsum) {
+  const int o = blockIdx.x * 256 + threadIdx.x;
+  if (o >= KH * W) return;
+  const int kh = o / W, c = o % W;
+  double acc = 0.0;
+  const long stride = long(KHMAX) * W;
+  const float *p = gpart + long(kh) * W + c;
+  const long n = long(B) * SPLIT;
+  long i = 0;
+  for (; i + 8 <= n; i += 8) {
+    float v[8];
+#pragma unroll
+    for (int u = 0; u < 8; ++u) v[u] = __ldg(p + (i + u) * stride);
+#pragma unroll
+    for (int u = 0; u < 8; ++u) acc += double(v[u]);
+  }
+  for (; i < n; ++i) acc += double(__ldg(p + i * stride));
+  gsum[o] = float(acc);
+}
+
 // The seeds' side (one CTA): merge the pool-backward partials over graphs and ranges, then
 // ∂q_kh, ∂W_k, ∂b_k, ∂Q1 -> ∂W_q, ∂b_q and ∂S = Σ_g ∂T1_g + W_qᵀ ∂Q1.
 template <int D>
@@ -1138,13 +1174,7 @@ __global__ void __launch_bounds__(DT) dec_seed_grads_kernel(const DecArgs a, con
   const DecLayout &L = a.L;
   const float *P = a.P;
   const float isq = rsqrtf(float(dh));
-  for (int o = t; o < KH * (D + 1); o += DT) {
-    const int kh = o / (D + 1), c = o % (D + 1);
-    double acc = 0.0;
-    for (int g = 0; g < a.B; ++g)
-      for (int q = 0; q < SPLIT; ++q) acc += double(gpart[((long(g) * SPLIT + q) * KHMAX + kh) * (D + 1) + c]);
-    Gs[kh][c] = float(acc);
-  }
+  for (int o = t; o < KH * (D + 1); o += DT) Gs[o / (D + 1)][o % (D + 1)] = gpart[o];   // merged (dec_gpart_reduce_kernel)
   for (int i = t; i < k * D; i += DT) S[i] = P[L.S + i];
   __syncthreads();
   warp_gemv(P + L.M1.Wq, D, D, D, S, D, k, Q, D, P + L.M1.bq, false);
@@ -1271,7 +1301,7 @@ int launch_set_decoder_bwd(occu_ctx *ctx, const DevCsr &csr, const float *hL, co
   const long RK = long(B) * k;
   const size_t f_rows = size_t(R_COUNT) * RK * D, f_pstat = size_t(B) * KHMAX * 2,
                f_pbar = size_t(B) * KH * D, f_u = size_t(B) * KHMAX * D,
-               f_ds = size_t(B) * SPLIT * KHMAX, f_gp = size_t(B) * SPLIT * KHMAX * (D + 1),
+               f_ds = size_t(B) * SPLIT * KHMAX, f_gp = (size_t(B) * SPLIT + 1) * KHMAX * (D + 1),
                f_h = size_t(RK) * D, f_x = size_t(RK) * D;
   if (ctx->ws.dbwd.ensure((f_rows + f_pstat + f_pbar + f_u + f_ds + f_gp + f_h + f_x) * 4) != cudaSuccess)
     return -int(cudaErrorMemoryAllocation);
@@ -1307,8 +1337,15 @@ int launch_set_decoder_bwd(occu_ctx *ctx, const DevCsr &csr, const float *hL, co
   OCCU_PROF_END(ctx);
   n += 2;
   OCCU_PROF_BEGIN(ctx, "dec_seed_grads", st);
-  if (D == 64) dec_seed_grads_kernel<64><<<1, DT, 0, st>>>(a, gp, rows + size_t(R_dT1) * RK * D, G);
-  else dec_seed_grads_kernel<128><<<1, DT, 0, st>>>(a, gp, rows + size_t(R_dT1) * RK * D, G);
+  {
+    // merged partials after the B·SPLIT raw ones (f_gp holds one extra [KHMAX][D + 1] slot)
+    float *gsum = gp + size_t(B) * SPLIT * KHMAX * (D + 1);
+    const int outs = k * cf.heads * (D + 1);
+    dec_gpart_reduce_kernel<<<(outs + 255) / 256, 256, 0, st>>>(gp, B, k * cf.heads, D + 1, gsum);
+    if (D == 64) dec_seed_grads_kernel<64><<<1, DT, 0, st>>>(a, gsum, rows + size_t(R_dT1) * RK * D, G);
+    else dec_seed_grads_kernel<128><<<1, DT, 0, st>>>(a, gsum, rows + size_t(R_dT1) * RK * D, G);
+    ++n;
+  }
   OCCU_PROF_END(ctx);
   ++n;
   // tail weight / bias / LayerNorm gradients: fixed-order reductions over the B·k rows
