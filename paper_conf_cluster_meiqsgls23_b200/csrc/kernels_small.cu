@@ -6,6 +6,18 @@
 // memory: one launch instead of ~9, no HBM round trips between steps.  FP32 on CUDA cores
 // (a few hundred kFLOP per layer; tensor-core tiles of 128 rows would be mostly padding).
 // Fixed summation orders (deterministic); P141-P151, P125.
+//
+// The three row-GEMMs of a layer run on the tensor cores through mma.sync m16n8k8 TF32 with
+// the 3xTF32 split (x = hi + lo, hi = x with its low 13 mantissa bits cleared: products
+// lo·hi + hi·lo + hi·hi accumulated in FP32, ~2^-20 relative — FP32-accurate for the 1e-4
+// contract), one warp per 16 rows x all D output channels (m16n8k8 measured at 512 MAC/cycle
+// on one SM, 4x the FP32 FMA rate; the SIMT register-blocked version was bound by shared-memory
+// wavefronts).  The step that follows each GEMM runs in its epilogue from the accumulator
+// fragments — LeakyReLU and the p = h̄·a_s, q = h̄·a_d dots (a2), σ(α z) (a3), the channel
+// softmax (a4) — with the row reductions as xor-shuffles over the 4 lanes that share a row.
+// Activation rows are padded to a stride that is an odd multiple of 4 words, so the fragment
+// loads (8 rows x 4 consecutive k) are conflict-free.  The a1 permutation is folded into the
+// layer-1 edge GEMM's row map (edge features staged in input order).
 #include <cuda_runtime.h>
 #include <math.h>
 #include <stdint.h>
@@ -17,8 +29,9 @@
 namespace occu {
 namespace {
 
-constexpr int SNMAX = 64, SEMAX = 128, SKMAX = 128, ST = 1024;   // 32 warps: latency hiding on one SM
+constexpr int SNMAX = 64, SEMAX = 128, SKMAX = 128, ST = 512;
 constexpr size_t SMEM_MAX = 220 * 1024;
+constexpr float LOG2E_S = 1.4426950408889634f;
 
 struct SmallArgs {
   const float *nf, *ef;                      // [N][F_n], [E][F_e] (input edge order)
@@ -26,7 +39,7 @@ struct SmallArgs {
   const float *P;                            // flat parameters
   size_t W_u[8], W_e[8], W_m[8], a_s[8], a_d[8];
   size_t W_1, b_1, w_2, b_2;
-  int L, F_n, F_e, d, d_h, B, N, E, mean, SK;     // SK = row stride of H / Ein (max width)
+  int L, F_n, F_e, d, d_h, B, N, E, mean, SK, KW;  // SK = row stride of H, KW = max GEMM K
   float slope;
   float *r, *c, *yhat;                       // [B][d], [B][d_h], [B]
 };
@@ -40,14 +53,15 @@ __device__ __forceinline__ float ex2_fast(float x) {
 
 #ifdef OCCU_SMALL_TIMING
 __device__ unsigned long long g_small_ts[64];
-#define STAMP(i) do { if (threadIdx.x == 0 && ts_n < 64) g_small_ts[ts_n++] = (unsigned long long)(i) << 56 | (clock64() & 0xFFFFFFFFFFFFFFull); } while (0)
+// the shared-memory read first: a BAR.SYNC blocks only at the next instruction that depends on
+// barrier-protected state, so the clock is read after the barrier has released
+#define STAMP(i) do { if (threadIdx.x == 0 && ts_n < 64) { const int dep_ = *reinterpret_cast<volatile int *>(ssm); \
+    g_small_ts[ts_n++] = ((unsigned long long)(i) << 56 | (clock64() & 0xFFFFFFFFFFFFFFull)) + (unsigned long long)(dep_ & 0); } } while (0)
 #else
 #define STAMP(i) do { } while (0)
 #endif
 
-// Global -> shared copies are cp.async (no register round trip, all in flight at once); weight
-// matrices [Nout][K] land row-major with row stride K + 4 through 16-byte copies (K % 4 == 0,
-// config validation), so the GEMM reads 4 consecutive k of one output with one 16-byte load.
+// Global -> shared copies are cp.async (no register round trip, all in flight at once).
 __device__ __forceinline__ void cpa4(void *dst, const void *src) {
   asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(static_cast<uint32_t>(__cvta_generic_to_shared(dst))),
                "l"(src) : "memory");
@@ -60,65 +74,189 @@ __device__ __forceinline__ void cpa_commit() { asm volatile("cp.async.commit_gro
 template <int N>
 __device__ __forceinline__ void cpa_wait() { asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory"); }
 
-__device__ __forceinline__ void stage_w(const float *__restrict__ W, int Nout, int K, float *Ws) {
-  const int K4 = K / 4;
-  if ((reinterpret_cast<uintptr_t>(W) & 15) == 0) {
-    for (int i = threadIdx.x; i < Nout * K4; i += ST) {
-      const int n = i / K4, k4 = i - n * K4;
-      cpa16(Ws + n * (K + 4) + 4 * k4, W + n * K + 4 * k4);
-    }
+// rows x cols floats (global row stride gld, shared row stride sld; cols % 4 == 0): warp per
+// row, lanes over 16-byte chunks — no integer division, and one out-of-line copy of the code
+// (the kernel body must stay small: it runs once per launch on one SM, so every instruction
+// is fetched cold from L2 once the body outgrows the 32 KB L1.5 instruction cache)
+__device__ __noinline__ void stage_rows(float *dst, int sld, const float *__restrict__ src, int gld,
+                                        int rows, int cols) {
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  if ((reinterpret_cast<uintptr_t>(src) & 15) == 0 && gld % 4 == 0 && sld % 4 == 0) {
+    for (int n = warp; n < rows; n += ST / 32)
+      for (int k = 4 * lane; k < cols; k += 128) cpa16(dst + n * sld + k, src + long(n) * gld + k);
   } else {
-    for (int i = threadIdx.x; i < Nout * K; i += ST) cpa4(Ws + (i / K) * (K + 4) + i % K, W + i);
+    for (int n = warp; n < rows; n += ST / 32)
+      for (int k = lane; k < cols; k += 32) cpa4(dst + n * sld + k, src + long(n) * gld + k);
   }
+}
+
+// weight matrix [Nout][K] -> shared [Nout][K + 4] (16-byte rows, bank-spread for the GEMM)
+__device__ __forceinline__ void stage_w(const float *__restrict__ W, int Nout, int K, float *Ws) {
+  stage_rows(Ws, K + 4, W, K, Nout, K);
   cpa_commit();
 }
 
-// Y[r][n] = Σ_k X[r][k] Ws[n][k] over rows r < R, outputs n < Nout (K % 4 == 0); thread per
-// (4-row block, output): one 16-byte weight load per 4 k serves four rows and the four input
-// loads are warp broadcasts (a warp = 32 outputs of one row block), so shared-memory traffic
-// is ~R·Nout·K bytes instead of 4x that; k ascending (fixed order).
-__device__ __forceinline__ void small_gemm(const float *X, int ldx, int R, int K, const float *Ws,
-                                           int Nout, float *Y, int ldy) {
-  const int ldw = K + 4, rblocks = (R + 3) / 4;
-  for (int i = threadIdx.x; i < rblocks * Nout; i += ST) {
-    const int rb = i / Nout, n = i - rb * Nout, r0 = rb * 4;
-    const float *w = Ws + n * ldw;
-    const float *x[4];
+constexpr int G_NODE = 0, G_EDGE = 1, G_GATE = 2;
+
+struct GemmEpi {
+  float slope;
+  const float *av;          // [2][D] a_s, a_d of the layer (G_NODE)
+  float *pq;                // [2][SNMAX] p, q (written by G_NODE, read by G_EDGE)
+  const int32_t *isrc, *idst;
+};
+
+__device__ __forceinline__ void split_tf32(float x, uint32_t &hi, uint32_t &lo) {
+  const uint32_t u = __float_as_uint(x) & 0xffffe000u;
+  hi = u;
+  lo = __float_as_uint(x - __uint_as_float(u));
+}
+__device__ __forceinline__ void mma_tf32(float (&c)[4], const uint32_t (&a)[4], uint32_t b0, uint32_t b1) {
+  asm("mma.sync.aligned.m16n8k8.row.col.f32.tf32.tf32.f32 {%0,%1,%2,%3}, {%4,%5,%6,%7}, {%8,%9}, {%0,%1,%2,%3};"
+      : "+f"(c[0]), "+f"(c[1]), "+f"(c[2]), "+f"(c[3])
+      : "r"(a[0]), "r"(a[1]), "r"(a[2]), "r"(a[3]), "r"(b0), "r"(b1));
+}
+
+// Y[r][n] = epi(Σ_k X[xrow(r)][k] Ws[n][k]) for r < R, n < D (row stride ldy; Ws row stride
+// K + 4).  Warp = m-tile of 16 rows, all D/8 n-tiles; fragment lane (g, t) = (lane/4, lane%4)
+// holds rows g, g+8, and output columns 8nt + 2t, 8nt + 2t + 1 of every n-tile.
+template <int D, int EPI>
+__device__ __forceinline__ void tgemm(const float *X, int ldx, const int32_t *xmap, int R, int K,
+                                      const float *Ws, float *Y, int ldy, const GemmEpi &ep) {
+  constexpr int NT = D / 8;
+  const int lane = threadIdx.x & 31, g = lane >> 2, tq = lane & 3;
+  const int MT = (R + 15) >> 4, ldw = K + 4;
+  for (int mt = threadIdx.x >> 5; mt < MT; mt += ST / 32) {
+    const int ra = mt * 16 + g, rb = ra + 8;
+    const bool va = ra < R, vb = rb < R;
+    const int ia = min(ra, R - 1), ib = min(rb, R - 1);
+    const float *xa = X + (xmap ? xmap[ia] : ia) * ldx, *xb = X + (xmap ? xmap[ib] : ib) * ldx;
+    float c[NT][4];
 #pragma unroll
-    for (int j = 0; j < 4; ++j) x[j] = X + min(r0 + j, R - 1) * ldx;
-    float a[4] = {0.f, 0.f, 0.f, 0.f};
-    for (int k = 0; k < K; k += 4) {
-      const float4 v = *reinterpret_cast<const float4 *>(w + k);
+    for (int nt = 0; nt < NT; ++nt) c[nt][0] = c[nt][1] = c[nt][2] = c[nt][3] = 0.f;
+#pragma unroll 1
+    for (int k0 = 0; k0 < K; k0 += 8) {
+      const int k1 = k0 + tq, k2 = k1 + 4;
+      const bool m1 = k1 < K, m2 = k2 < K;
+      uint32_t ah[4], al[4];
+      split_tf32(m1 ? xa[k1] : 0.f, ah[0], al[0]);
+      split_tf32(m1 ? xb[k1] : 0.f, ah[1], al[1]);
+      split_tf32(m2 ? xa[k2] : 0.f, ah[2], al[2]);
+      split_tf32(m2 ? xb[k2] : 0.f, ah[3], al[3]);
 #pragma unroll
-      for (int j = 0; j < 4; ++j) {
-        const float4 u = *reinterpret_cast<const float4 *>(x[j] + k);
-        a[j] = fmaf(u.w, v.w, fmaf(u.z, v.z, fmaf(u.y, v.y, fmaf(u.x, v.x, a[j]))));
+      for (int nt = 0; nt < NT; ++nt) {
+        const float *w = Ws + (nt * 8 + g) * ldw;
+        uint32_t bh0, bl0, bh1, bl1;
+        split_tf32(m1 ? w[k1] : 0.f, bh0, bl0);
+        split_tf32(m2 ? w[k2] : 0.f, bh1, bl1);
+        mma_tf32(c[nt], al, bh0, bh1);          // small terms first
+        mma_tf32(c[nt], ah, bl0, bl1);
+        mma_tf32(c[nt], ah, bh0, bh1);
       }
     }
+    if (EPI == G_NODE) {
+      // a2: h̄ = LReLU(.), p = h̄·a_s, q = h̄·a_d
+      float pa = 0.f, qa = 0.f, pb = 0.f, qb = 0.f;
 #pragma unroll
-    for (int j = 0; j < 4; ++j)
-      if (r0 + j < R) Y[(r0 + j) * ldy + n] = a[j];
+      for (int nt = 0; nt < NT; ++nt)
+#pragma unroll
+        for (int h = 0; h < 2; ++h) {
+          const int col = nt * 8 + 2 * tq + h;
+          const float oa = lrelu_s(c[nt][h], ep.slope), ob = lrelu_s(c[nt][2 + h], ep.slope);
+          c[nt][h] = oa;
+          c[nt][2 + h] = ob;
+          pa = fmaf(oa, ep.av[col], pa);
+          qa = fmaf(oa, ep.av[D + col], qa);
+          pb = fmaf(ob, ep.av[col], pb);
+          qb = fmaf(ob, ep.av[D + col], qb);
+        }
+#pragma unroll
+      for (int o = 1; o <= 2; o <<= 1) {
+        pa += __shfl_xor_sync(0xffffffffu, pa, o);
+        qa += __shfl_xor_sync(0xffffffffu, qa, o);
+        pb += __shfl_xor_sync(0xffffffffu, pb, o);
+        qb += __shfl_xor_sync(0xffffffffu, qb, o);
+      }
+      if (tq == 0) {
+        if (va) { ep.pq[ra] = pa; ep.pq[SNMAX + ra] = qa; }
+        if (vb) { ep.pq[rb] = pb; ep.pq[SNMAX + rb] = qb; }
+      }
+    } else if (EPI == G_EDGE) {
+      // a3: e' = σ(α z), α = p[src] + q[dst]
+      const float ala = ep.pq[ep.isrc[ia]] + ep.pq[SNMAX + ep.idst[ia]];
+      const float alb = ep.pq[ep.isrc[ib]] + ep.pq[SNMAX + ep.idst[ib]];
+#pragma unroll
+      for (int nt = 0; nt < NT; ++nt)
+#pragma unroll
+        for (int h = 0; h < 2; ++h) {
+          c[nt][h] = __fdividef(1.f, 1.f + ex2_fast(-ala * c[nt][h] * LOG2E_S));
+          c[nt][2 + h] = __fdividef(1.f, 1.f + ex2_fast(-alb * c[nt][2 + h] * LOG2E_S));
+        }
+    } else {
+      // a4: g = softmax over the D channels of the logits (rows g and g+8)
+      float ma = -INFINITY, mb = -INFINITY;
+#pragma unroll
+      for (int nt = 0; nt < NT; ++nt) {
+        ma = fmaxf(ma, fmaxf(c[nt][0], c[nt][1]));
+        mb = fmaxf(mb, fmaxf(c[nt][2], c[nt][3]));
+      }
+#pragma unroll
+      for (int o = 1; o <= 2; o <<= 1) {
+        ma = fmaxf(ma, __shfl_xor_sync(0xffffffffu, ma, o));
+        mb = fmaxf(mb, __shfl_xor_sync(0xffffffffu, mb, o));
+      }
+      float sa = 0.f, sb = 0.f;
+#pragma unroll
+      for (int nt = 0; nt < NT; ++nt)
+#pragma unroll
+        for (int h = 0; h < 2; ++h) {
+          c[nt][h] = ex2_fast((c[nt][h] - ma) * LOG2E_S);
+          c[nt][2 + h] = ex2_fast((c[nt][2 + h] - mb) * LOG2E_S);
+          sa += c[nt][h];
+          sb += c[nt][2 + h];
+        }
+#pragma unroll
+      for (int o = 1; o <= 2; o <<= 1) {
+        sa += __shfl_xor_sync(0xffffffffu, sa, o);
+        sb += __shfl_xor_sync(0xffffffffu, sb, o);
+      }
+      const float inva = 1.f / sa, invb = 1.f / sb;
+#pragma unroll
+      for (int nt = 0; nt < NT; ++nt)
+#pragma unroll
+        for (int h = 0; h < 2; ++h) {
+          c[nt][h] *= inva;
+          c[nt][2 + h] *= invb;
+        }
+    }
+#pragma unroll
+    for (int nt = 0; nt < NT; ++nt) {
+      const int col = nt * 8 + 2 * tq;
+      if (va) *reinterpret_cast<float2 *>(Y + ra * ldy + col) = make_float2(c[nt][0], c[nt][1]);
+      if (vb) *reinterpret_cast<float2 *>(Y + rb * ldy + col) = make_float2(c[nt][2], c[nt][3]);
+    }
   }
 }
 
+template <int D>
 __global__ void __launch_bounds__(ST, 1) small_forward_kernel(const SmallArgs a) {
-  extern __shared__ float ssm[];
-  const int d = a.d, N = a.N, E = a.E, SK = a.SK;
+  extern __shared__ __align__(16) float ssm[];
+  constexpr int LD = D + 4;                    // row stride of h̄ and the edge arrays (odd multiple of 4 words)
+  const int N = a.N, E = a.E, SK = a.SK, dh = a.d_h, B = a.B;
   float *H = ssm;                              // [N][SK] layer input h
-  float *Hb = H + N * SK;                      // [N][d]  h̄
-  float *pq = Hb + N * d;                      // [2][SNMAX]  p, q
-  float *E0 = pq + 2 * SNMAX;                  // [E][F_e] layer-1 edge input (in-CSR order)
-  float *Ev = E0 + E * a.F_e;                  // [E][d]  z / logits / gates
-  float *Ea = Ev + E * d;                      // [E][d]  e' (ping)
-  float *Eb = Ea + E * d;                      // [E][d]  e' (pong)
-  float *Wa = Eb + E * d;                      // [d][SK + 4] weight slot A (W_u, W_m)
-  float *Wb = Wa + d * (SK + 4);               // [d][SK + 4] weight slot B (W_e)
-  float *W1s = Wb + d * (SK + 4);              // [d_h][d] head W_1, then b_1 [d_h], w_2 [d_h]
-  float *Rs = W1s + a.d_h * d + 2 * a.d_h;     // [B][d] readout
-  float *Cs = Rs + a.B * d;                    // [B][d_h] head hidden
-  float *Av = Cs + a.B * a.d_h;                // [L][2][d] attention vectors a_s, a_d
-  int32_t *cs = reinterpret_cast<int32_t *>(Av + a.L * 2 * d);
-  int32_t *iptr = cs, *isrc = cs + (N + 1), *idst = isrc + E, *ieid = idst + E;
+  float *Hb = H + N * SK;                      // [N][LD] h̄
+  float *pq = Hb + N * LD;                     // [2][SNMAX]  p, q
+  float *Ef = pq + 2 * SNMAX;                  // [E][F_e] layer-1 edge input (INPUT edge order)
+  float *Ev = Ef + E * a.F_e;                  // [E][LD] gates
+  float *Ea = Ev + E * LD;                     // [E][LD] e' (ping)
+  float *Eb = Ea + E * LD;                     // [E][LD] e' (pong)
+  float *Wa = Eb + E * LD;                     // [D][K + 4] weight slot A (W_u, W_m)
+  float *Wb = Wa + D * (a.KW + 4);             // [D][K + 4] weight slot B (W_e)
+  float *W1s = Wb + D * (a.KW + 4);            // [d_h][D + 4] head W_1, then b_1, w_2 [d_h], b_2
+  float *Rs = W1s + dh * (D + 4) + 2 * dh + 4; // [B][D] readout
+  float *Cs = Rs + B * D;                      // [B][d_h] head hidden
+  float *Av = Cs + B * dh;                     // [L][2][D] attention vectors a_s, a_d
+  int32_t *cs = reinterpret_cast<int32_t *>(Av + a.L * 2 * D);
+  int32_t *iptr = cs, *isrc = cs + (N + 1), *idst = isrc + E, *ieid = idst + E, *noff = ieid + E;
   const int t = threadIdx.x, warp = t >> 5, lane = t & 31;
 #ifdef OCCU_SMALL_TIMING
   int ts_n = 0;
@@ -126,162 +264,166 @@ __global__ void __launch_bounds__(ST, 1) small_forward_kernel(const SmallArgs a)
   STAMP(0);
   pdl_trigger();
   pdl_wait();
-  // a1: CSR, node features, first layer's weights; then the in-CSR-ordered edge features
+#ifdef OCCU_SMALL_TIMING
+  for (int rep = 0; rep < 2; ++rep) {        // probe: the second pass runs with a warm i-cache
+  __syncthreads();
+#endif
+  // group 0: CSR, graph offsets, node and edge features, every layer's attention vectors; then
+  // the first layer's weights (one group each) and the head's parameters
   for (int i = t; i <= N; i += ST) cpa4(iptr + i, a.in_ptr + i);
+  for (int i = t; i <= B; i += ST) cpa4(noff + i, a.node_off + i);
   for (int i = t; i < E; i += ST) {
     cpa4(isrc + i, a.in_src + i);
     cpa4(idst + i, a.in_dst + i);
     cpa4(ieid + i, a.in_eid + i);
   }
-  for (int i = t; i < N * a.F_n; i += ST) cpa4(H + (i / a.F_n) * SK + i % a.F_n, a.nf + i);
-  // the attention vectors of every layer and the head's parameters ride in the first group
-  for (int i = t; i < a.L * 2 * d; i += ST) {
-    const int l = i / (2 * d), j = i % (2 * d);
-    cpa4(Av + i, a.P + (j < d ? a.a_s[l] + j : a.a_d[l] + j - d));
-  }
-  for (int i = t; i < a.d_h * d; i += ST) cpa4(W1s + i, a.P + a.W_1 + i);
-  for (int i = t; i < a.d_h; i += ST) {
-    cpa4(W1s + a.d_h * d + i, a.P + a.b_1 + i);
-    cpa4(W1s + a.d_h * d + a.d_h + i, a.P + a.w_2 + i);
+  stage_rows(H, SK, a.nf, a.F_n, N, a.F_n);
+  stage_rows(Ef, a.F_e, a.ef, a.F_e, E, a.F_e);
+  for (int i = t; i < a.L * 2 * D; i += ST) {
+    const int l = i / (2 * D), j = i % (2 * D);
+    cpa4(Av + i, a.P + (j < D ? a.a_s[l] + j : a.a_d[l] + j - D));
   }
   cpa_commit();
-  stage_w(a.P + a.W_u[0], d, a.F_n, Wa);
-  stage_w(a.P + a.W_e[0], d, a.F_e, Wb);
-  cpa_wait<2>();                               // CSR + node features
-  __syncthreads(); STAMP(1);
-  for (int i = t; i < E * a.F_e; i += ST) {
-    const int k = i / a.F_e, c = i % a.F_e;
-    cpa4(E0 + i, a.ef + size_t(ieid[k]) * a.F_e + c);
+  stage_w(a.P + a.W_u[0], D, a.F_n, Wa);
+  stage_w(a.P + a.W_e[0], D, a.F_e, Wb);
+  // the head's parameters: last group of the prologue (needed only after the last layer)
+  stage_rows(W1s, D + 4, a.P + a.W_1, D, dh, D);
+  float *b1s = W1s + dh * (D + 4), *w2s = b1s + dh;
+  for (int i = t; i < dh; i += ST) {
+    cpa4(b1s + i, a.P + a.b_1 + i);
+    cpa4(w2s + i, a.P + a.w_2 + i);
   }
-  cpa_commit();                                // groups in flight: W_u, W_e, E0
-  int K = a.F_n, Ke = a.F_e;
-  const float *Ein = E0;
+  if (t == 0) cpa4(w2s + dh, a.P + a.b_2);
+  cpa_commit();
+  int K = a.F_n;
+  const float *Ein = Ef;
   int lde = a.F_e;
   float *Eout = Ea;
+  GemmEpi ep{a.slope, nullptr, pq, isrc, idst};
   for (int l = 0; l < a.L; ++l) {
     const float *P = a.P;
-    // a2: h̄ = LReLU(h W_uᵀ); p = h̄·a_s, q = h̄·a_d          (groups: W_u, W_e[, E0])
-    // layer 0: W_u0 is the second of four groups (CSR + H, W_u0, W_e0, E0); later layers:
-    // W_u(l) is the most recent group (issued after W_e(l)), so everything must land
-    if (l == 0) cpa_wait<2>(); else cpa_wait<0>();
+    // a2 (groups pending: layer 0 — group 0, W_u, W_e; later — W_e(l), W_u(l))
+    if (l == 0) cpa_wait<2>(); else cpa_wait<0>();       // layer 0: W_e0 and the head may pend
+    __syncthreads(); STAMP(1);
+    ep.av = Av + l * 2 * D;
+    tgemm<D, G_NODE>(H, SK, nullptr, N, K, Wa, Hb, LD, ep);
     __syncthreads(); STAMP(2);
-    small_gemm(H, SK, N, K, Wa, d, Hb, d);
+    stage_w(P + a.W_m[l], D, D, Wa);           // slot A: W_m (W_u consumed)
+    // a3 (+ a1 on layer 1: rows of the input-order edge features through in_eid)
+    if (l == 0) cpa_wait<2>(); else cpa_wait<1>();       // W_m pends (layer 0: and the head)
     __syncthreads(); STAMP(3);
-    stage_w(P + a.W_m[l], d, d, Wa);           // slot A: W_m (W_u consumed)
-    for (int i = t; i < N * d; i += ST) Hb[i] = lrelu_s(Hb[i], a.slope);
+    tgemm<D, G_EDGE>(Ein, lde, l == 0 ? ieid : nullptr, E, l == 0 ? a.F_e : D, Wb, Eout, LD, ep);
     __syncthreads(); STAMP(4);
-    for (int u = warp; u < N; u += ST / 32) {
-      float ps = 0.f, qs = 0.f;
-      for (int c = lane; c < d; c += 32) {
-        ps = fmaf(Hb[u * d + c], Av[l * 2 * d + c], ps);
-        qs = fmaf(Hb[u * d + c], Av[l * 2 * d + d + c], qs);
-      }
-#pragma unroll
-      for (int o = 16; o > 0; o >>= 1) {
-        ps += __shfl_xor_sync(0xffffffffu, ps, o);
-        qs += __shfl_xor_sync(0xffffffffu, qs, o);
-      }
-      if (lane == 0) {
-        pq[u] = ps;
-        pq[SNMAX + u] = qs;
-      }
-    }
-    // a3: z = e_in W_eᵀ, e' = σ(α z), α = p[src] + q[dst]     (groups: W_e[, E0], W_m)
-    cpa_wait<1>();
-    __syncthreads(); STAMP(5);
-    small_gemm(Ein, lde, E, Ke, Wb, d, Ev, d);
-    __syncthreads(); STAMP(6);
-    if (l + 1 < a.L) stage_w(P + a.W_e[l + 1], d, d, Wb);      // slot B: next W_e
-    for (int i = t; i < E * d; i += ST) {
-      const int k = i / d;
-      const float al = pq[isrc[k]] + pq[SNMAX + idst[k]];
-      Eout[i] = __fdividef(1.f, 1.f + ex2_fast(-al * Ev[i] * 1.4426950408889634f));
-    }
-    // a4: logits W_m e', softmax over the d channels (warp per edge)
+    if (l + 1 < a.L) stage_w(P + a.W_e[l + 1], D, D, Wb);      // slot B: next W_e
+    // a4
     if (l + 1 < a.L) cpa_wait<1>(); else cpa_wait<0>();
-    __syncthreads(); STAMP(7);
-    small_gemm(Eout, d, E, d, Wa, d, Ev, d);
-    __syncthreads(); STAMP(8);
-    if (l + 1 < a.L) stage_w(P + a.W_u[l + 1], d, d, Wa);      // slot A: next W_u
-    for (int k = warp; k < E; k += ST / 32) {
-      float m = -INFINITY;
-      for (int c = lane; c < d; c += 32) m = fmaxf(m, Ev[k * d + c]);
-#pragma unroll
-      for (int o = 16; o > 0; o >>= 1) m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, o));
-      float s = 0.f;
-      for (int c = lane; c < d; c += 32) {
-        const float x = ex2_fast((Ev[k * d + c] - m) * 1.4426950408889634f);
-        Ev[k * d + c] = x;
-        s += x;
-      }
-#pragma unroll
-      for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
-      const float inv = 1.f / s;
-      for (int c = lane; c < d; c += 32) Ev[k * d + c] *= inv;
-    }
-    __syncthreads(); STAMP(9);
+    __syncthreads(); STAMP(5);
+    tgemm<D, G_GATE>(Eout, LD, nullptr, E, D, Wa, Ev, LD, ep);
+    __syncthreads(); STAMP(6);
+    if (l + 1 < a.L) stage_w(P + a.W_u[l + 1], D, D, Wa);      // slot A: next W_u
     // a5/a6: h[t] = LReLU(Σ_{k∈seg(t)} g_k ⊙ h̄[s_k]) (÷ deg for MEAN), ascending k
-    for (int i = t; i < N * d; i += ST) {
-      const int v = i / d, c = i % d;
+    for (int i = t; i < N * (D / 4); i += ST) {
+      const int v = i / (D / 4), c = 4 * (i % (D / 4));
       const int k0 = iptr[v], k1 = iptr[v + 1];
-      float acc = 0.f;
-      for (int k = k0; k < k1; ++k) acc = fmaf(Ev[k * d + c], Hb[isrc[k] * d + c], acc);
-      if (a.mean) acc /= float(k1 > k0 ? k1 - k0 : 1);
-      H[v * SK + c] = lrelu_s(acc, a.slope);
+      float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
+      for (int k = k0; k < k1; ++k) {
+        const float4 g = *reinterpret_cast<const float4 *>(Ev + k * LD + c);
+        const float4 h = *reinterpret_cast<const float4 *>(Hb + isrc[k] * LD + c);
+        acc.x = fmaf(g.x, h.x, acc.x);
+        acc.y = fmaf(g.y, h.y, acc.y);
+        acc.z = fmaf(g.z, h.z, acc.z);
+        acc.w = fmaf(g.w, h.w, acc.w);
+      }
+      if (a.mean) {
+        const float dg = float(k1 > k0 ? k1 - k0 : 1);
+        acc.x /= dg; acc.y /= dg; acc.z /= dg; acc.w /= dg;
+      }
+      *reinterpret_cast<float4 *>(H + v * SK + c) =
+          make_float4(lrelu_s(acc.x, a.slope), lrelu_s(acc.y, a.slope), lrelu_s(acc.z, a.slope), lrelu_s(acc.w, a.slope));
     }
-    __syncthreads(); STAMP(10);
+    __syncthreads(); STAMP(7);
     Ein = Eout;                                // e' feeds the next layer (ping-pong)
-    lde = d;
+    lde = LD;
     Eout = Eout == Ea ? Eb : Ea;
-    K = d;
-    Ke = d;
+    K = D;
   }
-  // a7: per-graph mean readout (shared memory); a8: head, warp per hidden unit (lanes over the
-  // d channels, fixed butterfly), then warp per graph for the final dot
-  for (int i = t; i < a.B * d; i += ST) {
-    const int b = i / d, c = i % d;
-    const int u0 = __ldg(a.node_off + b), u1 = __ldg(a.node_off + b + 1);
-    float s = 0.f;
-    for (int u = u0; u < u1; ++u) s += H[u * SK + c];
-    Rs[i] = s / float(u1 - u0);
-    a.r[i] = Rs[i];
-  }
-  __syncthreads(); STAMP(11);
-  for (int o = warp; o < a.B * a.d_h; o += ST / 32) {
-    const int b = o / a.d_h, n = o % a.d_h;
-    float s = 0.f;
-    for (int c = lane; c < d; c += 32) s = fmaf(W1s[n * d + c], Rs[b * d + c], s);
+  // a7: per-graph mean readout (ascending nodes); a8: head, thread per hidden unit (W_1 rows
+  // padded to D + 1: conflict-free), then warp per graph for the final dot
+  for (int i = t; i < B * (D / 4); i += ST) {
+    const int b = i / (D / 4), c = 4 * (i % (D / 4));
+    const int u0 = noff[b], u1 = noff[b + 1];
+    float4 s[4];
 #pragma unroll
-    for (int q = 16; q > 0; q >>= 1) s += __shfl_xor_sync(0xffffffffu, s, q);
-    if (lane == 0) {
-      s += W1s[a.d_h * d + n];
-      Cs[o] = s;
-      a.c[o] = s;
-    }
+    for (int q = 0; q < 4; ++q) s[q] = make_float4(0.f, 0.f, 0.f, 0.f);
+    for (int u = u0; u < u1; u += 4)
+#pragma unroll
+      for (int q = 0; q < 4; ++q)
+        if (u + q < u1) {
+          const float4 h = *reinterpret_cast<const float4 *>(H + (u + q) * SK + c);
+          s[q].x += h.x; s[q].y += h.y; s[q].z += h.z; s[q].w += h.w;
+        }
+    const float n = float(u1 - u0);
+    float4 o;
+    o.x = ((s[0].x + s[1].x) + (s[2].x + s[3].x)) / n;
+    o.y = ((s[0].y + s[1].y) + (s[2].y + s[3].y)) / n;
+    o.z = ((s[0].z + s[1].z) + (s[2].z + s[3].z)) / n;
+    o.w = ((s[0].w + s[1].w) + (s[2].w + s[3].w)) / n;
+    *reinterpret_cast<float4 *>(Rs + b * D + c) = o;
+    *reinterpret_cast<float4 *>(a.r + b * D + c) = o;
   }
-  __syncthreads(); STAMP(12);
-  for (int b = warp; b < a.B; b += ST / 32) {
+  __syncthreads(); STAMP(8);
+  for (int o = t; o < B * dh; o += ST) {
+    const int b = o / dh, n = o % dh;
+    const float *w = W1s + n * (D + 4), *rr = Rs + b * D;
+    float s4[4] = {0.f, 0.f, 0.f, 0.f};
+#pragma unroll 4
+    for (int c = 0; c < D; c += 4) {
+      const float4 wv = *reinterpret_cast<const float4 *>(w + c), rv = *reinterpret_cast<const float4 *>(rr + c);
+      s4[0] = fmaf(wv.x, rv.x, s4[0]);
+      s4[1] = fmaf(wv.y, rv.y, s4[1]);
+      s4[2] = fmaf(wv.z, rv.z, s4[2]);
+      s4[3] = fmaf(wv.w, rv.w, s4[3]);
+    }
+    const float s = ((s4[0] + s4[1]) + (s4[2] + s4[3])) + b1s[n];
+    Cs[o] = s;
+    a.c[o] = s;
+  }
+  __syncthreads(); STAMP(9);
+  for (int b = warp; b < B; b += ST / 32) {
     float s = 0.f;
-    for (int n = lane; n < a.d_h; n += 32) s = fmaf(W1s[a.d_h * d + a.d_h + n], lrelu_s(Cs[b * a.d_h + n], a.slope), s);
+    for (int n = lane; n < dh; n += 32) s = fmaf(w2s[n], lrelu_s(Cs[b * dh + n], a.slope), s);
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
-    if (lane == 0) a.yhat[b] = s + __ldg(a.P + a.b_2);
+    if (lane == 0) a.yhat[b] = s + w2s[dh];
   }
+#ifdef OCCU_SMALL_TIMING
+  }
+#endif
 }
 
 }  // namespace
 
+// H row stride: the widest layer input, rounded up to an odd multiple of 4 words (the MMA
+// fragment loads of 8 rows x 4 consecutive k then hit 32 distinct banks)
+static int small_sk(const occu_config &c) {
+  int sk = (std::max(c.F_n, std::max(c.F_e, c.d)) + 3) / 4 * 4;
+  if ((sk / 4) % 2 == 0) sk += 4;
+  return sk;
+}
+static int small_kw(const occu_config &c) { return std::max(c.F_n, std::max(c.F_e, c.d)); }
+
 static size_t small_smem(const occu_config &c, const DevCsr &csr) {
-  const int sk = std::max(c.F_n, std::max(c.F_e, c.d));
-  return size_t(csr.N * sk + csr.N * c.d + 2 * SNMAX + csr.E * c.F_e + 3 * csr.E * c.d +
-                2 * c.d * (sk + 4) + c.d_h * c.d + 2 * c.d_h + csr.B * (c.d + c.d_h) + c.L * 2 * c.d + (csr.N + 1) + 3 * csr.E) * 4;
+  const int sk = small_sk(c), ld = c.d + 4;
+  return size_t(csr.N * sk + csr.N * ld + 2 * SNMAX + csr.E * c.F_e + 3 * csr.E * ld +
+                2 * c.d * (small_kw(c) + 4) + c.d_h * (c.d + 4) + 2 * c.d_h + 4 + csr.B * (c.d + c.d_h) +
+                c.L * 2 * c.d + (csr.N + 1) + 3 * csr.E + (csr.B + 1)) * 4;
 }
 
 bool small_forward_ok(const occu_ctx *ctx, const DevCsr &csr) {
   const occu_config &c = ctx->cfg;
   return c.prec == OCCU_FP32 && c.msg == OCCU_MSG_CHANNEL_SOFTMAX && c.readout == OCCU_READOUT_MEAN &&
-         c.graphormer == 0 && c.L <= 8 && csr.N >= 1 && csr.N <= SNMAX && csr.E <= SEMAX &&
-         c.F_n <= SKMAX && c.F_e <= SKMAX && c.d <= SKMAX && small_smem(c, csr) <= SMEM_MAX;
+         c.graphormer == 0 && c.L <= 8 && (c.d == 64 || c.d == 128) && csr.N >= 1 && csr.N <= SNMAX &&
+         csr.E <= SEMAX && c.F_n <= SKMAX && c.F_e <= SKMAX && small_smem(c, csr) <= SMEM_MAX;
 }
 
 int launch_small_forward(const occu_ctx *ctx, const DevCsr &csr, const float *nf, const float *ef,
@@ -300,12 +442,18 @@ int launch_small_forward(const occu_ctx *ctx, const DevCsr &csr, const float *nf
   a.L = c.L; a.F_n = c.F_n; a.F_e = c.F_e; a.d = c.d; a.d_h = c.d_h;
   a.B = csr.B; a.N = csr.N; a.E = csr.E; a.mean = c.aggr == OCCU_AGGR_MEAN;
   a.slope = c.slope;
-  a.SK = std::max(c.F_n, std::max(c.F_e, c.d));   // H row stride; W staged with K + 1
+  a.SK = small_sk(c);
+  a.KW = small_kw(c);
   a.r = r; a.c = cvec; a.yhat = yhat;
   const size_t smem = small_smem(c, csr);
-  cudaFuncSetAttribute(small_forward_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
   OCCU_PROF_BEGIN(ctx, "small_forward", st);
-  small_forward_kernel<<<1, ST, smem, st>>>(a);
+  if (c.d == 64) {
+    cudaFuncSetAttribute(small_forward_kernel<64>, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
+    small_forward_kernel<64><<<1, ST, smem, st>>>(a);
+  } else {
+    cudaFuncSetAttribute(small_forward_kernel<128>, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
+    small_forward_kernel<128><<<1, ST, smem, st>>>(a);
+  }
   OCCU_PROF_END(ctx);
   const cudaError_t e = cudaGetLastError();
   return e == cudaSuccess ? 1 : -int(e);
