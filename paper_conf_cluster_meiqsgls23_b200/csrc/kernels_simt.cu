@@ -999,13 +999,18 @@ __global__ void __launch_bounds__(NT) gather_segsoftmax_kernel(
 // flight), then the warp walks the edges four at a time with the e' / de rows of the four in
 // flight; lane = D/32 channels (coalesced rows), W_e's columns for the lane's channels live in
 // registers; the dot is a fixed-order butterfly.  BF: e' rows are BF16 (OCCU_BF16 training).
+// FUSEW (KM = Ke = 4): the layer's weight gradient dW_e = DZᵀ e0 is accumulated here as well
+// (lane = its channels x the Ke features, FP32 over the warp's edges, warps combined in fixed
+// order per block) into per-block partials dwe_part[block][D][Ke], reduced in block order by
+// the layer's multi_reduce — DZ is not read back by a weight-gradient kernel.
 // ---------------------------------------------------------------------------
-template <int D, int KM, bool BF>
+template <int D, int KM, bool BF, bool FUSEW = false>
 __global__ void __launch_bounds__(NT) edge_bwd_small_kernel(
     const float *__restrict__ e0, int Ke, const void *__restrict__ e, const float *__restrict__ de,
     const float *__restrict__ W_e, const float *__restrict__ p, const float *__restrict__ q,
     const int32_t *__restrict__ in_src, const int32_t *__restrict__ in_dst, int E,
-    float *__restrict__ DZ, float *__restrict__ dalpha) {
+    float *__restrict__ DZ, float *__restrict__ dalpha, float *__restrict__ dwe_part = nullptr) {
+  static_assert(!FUSEW || KM == 4, "fused dW_e: Ke = 4 only");
   constexpr int V = D / 32;
   constexpr int G = 4;
   constexpr float L2E = 1.4426950408889634f;
@@ -1015,6 +1020,11 @@ __global__ void __launch_bounds__(NT) edge_bwd_small_kernel(
   for (int j = 0; j < KM; ++j)
 #pragma unroll
     for (int c = 0; c < V; ++c) w[j][c] = j < Ke ? __ldg(W_e + long(lane * V + c) * Ke + j) : 0.f;
+  float gw[FUSEW ? V : 1][FUSEW ? KM : 1];
+#pragma unroll
+  for (int c = 0; c < (FUSEW ? V : 1); ++c)
+#pragma unroll
+    for (int j = 0; j < (FUSEW ? KM : 1); ++j) gw[c][j] = 0.f;
   const long nwarps = long(gridDim.x) * (NT / 32);
   for (long k0 = (blockIdx.x * long(NT / 32) + threadIdx.x / 32) * 32; k0 < E; k0 += nwarps * 32) {
     const int cnt = int(min(32L, E - k0));
@@ -1047,12 +1057,13 @@ __global__ void __launch_bounds__(NT) edge_bwd_small_kernel(
         if (jb + u >= cnt) break;                       // warp-uniform
         const int kk = jb + u;
         const float a = __shfl_sync(0xffffffffu, al, kk);
-        float z[V];
+        float z[V], xs[KM];
 #pragma unroll
         for (int c = 0; c < V; ++c) z[c] = 0.f;
 #pragma unroll
         for (int j = 0; j < KM; ++j) {
           const float x = __shfl_sync(0xffffffffu, ev[j], kk);
+          xs[j] = x;
 #pragma unroll
           for (int c = 0; c < V; ++c) z[c] = fmaf(w[j][c], x, z[c]);
         }
@@ -1071,9 +1082,29 @@ __global__ void __launch_bounds__(NT) edge_bwd_small_kernel(
         for (int off = 16; off > 0; off >>= 1) dot += __shfl_xor_sync(0xffffffffu, dot, off);
         store_row<V>(DZ + (k0 + kk) * D + lane * V, o);
         if (lane == kk) dal_mine = float(dot);
+        if constexpr (FUSEW) {
+#pragma unroll
+          for (int c = 0; c < V; ++c)
+#pragma unroll
+            for (int j = 0; j < KM; ++j) gw[c][j] = fmaf(o[c], xs[j], gw[c][j]);    // DZᵀ e0, edge order
+        }
       }
     }
     if (lane < cnt) dalpha[k0 + lane] = dal_mine;
+  }
+  if constexpr (FUSEW) {
+    __shared__ float red[NT / 32][D * KM];
+    const int wl = threadIdx.x / 32;
+#pragma unroll
+    for (int c = 0; c < V; ++c)
+#pragma unroll
+      for (int j = 0; j < KM; ++j) red[wl][(lane * V + c) * KM + j] = gw[c][j];
+    __syncthreads();
+    for (int o = threadIdx.x; o < D * KM; o += NT) {
+      double acc = 0.0;
+      for (int w2 = 0; w2 < NT / 32; ++w2) acc += red[w2][o];
+      dwe_part[long(blockIdx.x) * D * KM + o] = float(acc);
+    }
   }
 }
 
@@ -2301,6 +2332,10 @@ static int backward_layer_impl(occu_ctx *ctx, const DevCsr &csr, const BwdLayerA
   const bool in_bf = bf && i > 0;           // h_in, e_in of layer 1 are the FP32 inputs
   if ((bf || cf.msg == OCCU_MSG_NEIGHBOR_SOFTMAX) && !(tc && a.g)) return -int(cudaErrorInvalidValue);
   int r;
+  if (w.partial.ensure(3 * WG_SLOT_FLOATS * 4) != cudaSuccess) return -int(cudaErrorMemoryAllocation);
+  float *slot = w.partial.as<float>();
+  static const bool fuse_we = !getenv("OCCU_NO_FUSE_WE");   // A/B switch: dW_e in the layer-1 edge backward
+  int we_blocks = 0;                        // > 0: dW_e partials already written by edge_bwd_small
   // the streaming gate backward (saved gates) leaves MG = dA[t] ⊙ g to the node backward
   const bool mg_from_g = tc && a.g && !getenv("OCCU_NODE_BWD_V1");
   float *MGo = mg_from_g ? nullptr : w.MG.as<float>();
@@ -2353,7 +2388,12 @@ static int backward_layer_impl(occu_ctx *ctx, const DevCsr &csr, const BwdLayerA
       const int eg = grid_for((long(csr.E) + 31) / 32, NT / 32, 8 * sms);
 #define OCCU_EBS_ARGS a.e_in, a.Ke, a.e, de, P + L.W_e[i], a.p, a.q, csr.in_src, csr.in_dst, csr.E, \
     w.DZ.as<float>(), w.dalpha.as<float>()
-      if (a.Ke <= 4) {
+      if (a.Ke == 4 && fuse_we) {
+        // layer 1 with F_e = 4: dW_e accumulated here (per-block partials in the W_e slot)
+        if (bf) edge_bwd_small_kernel<D, 4, true, true><<<eg, NT, 0, st>>>(OCCU_EBS_ARGS, slot + WG_SLOT_FLOATS);
+        else edge_bwd_small_kernel<D, 4, false, true><<<eg, NT, 0, st>>>(OCCU_EBS_ARGS, slot + WG_SLOT_FLOATS);
+        we_blocks = eg;
+      } else if (a.Ke <= 4) {
         if (bf) edge_bwd_small_kernel<D, 4, true><<<eg, NT, 0, st>>>(OCCU_EBS_ARGS);
         else edge_bwd_small_kernel<D, 4, false><<<eg, NT, 0, st>>>(OCCU_EBS_ARGS);
       } else {
@@ -2421,13 +2461,15 @@ static int backward_layer_impl(occu_ctx *ctx, const DevCsr &csr, const BwdLayerA
   // sums into per-GEMM slots, all of the layer's split reductions in one launch
   ReduceJobs rj{};
   rj.j[rj.count++] = ReduceJob{da_part, G + L.a_s[i], long(2 * D), nb_blocks};
-  if (w.partial.ensure(3 * WG_SLOT_FLOATS * 4) != cudaSuccess) return -int(cudaErrorMemoryAllocation);
-  float *slot = w.partial.as<float>();
   if ((r = wgrad_deferred(ctx, w.DV.as<float>(), D, a.e, D, csr.E, G + L.W_m[i], st, bf, rj, slot)) < 0) return r;
   n += r;
-  if ((r = wgrad_deferred(ctx, w.DZ.as<float>(), D, a.e_in, a.Ke, csr.E, G + L.W_e[i], st, in_bf, rj,
-                          slot + WG_SLOT_FLOATS)) < 0) return r;
-  n += r;
+  if (we_blocks > 0) {
+    rj.j[rj.count++] = ReduceJob{slot + WG_SLOT_FLOATS, G + L.W_e[i], long(D) * a.Ke, we_blocks};
+  } else {
+    if ((r = wgrad_deferred(ctx, w.DZ.as<float>(), D, a.e_in, a.Ke, csr.E, G + L.W_e[i], st, in_bf, rj,
+                            slot + WG_SLOT_FLOATS)) < 0) return r;
+    n += r;
+  }
   if ((r = wgrad_deferred(ctx, w.dP.as<float>(), D, a.h_in, a.K, csr.N, G + L.W_u[i], st, in_bf, rj,
                           slot + 2 * WG_SLOT_FLOATS)) < 0) return r;
   n += r;
