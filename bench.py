@@ -210,7 +210,8 @@ def train_algorithmic_bytes(N, E, B, d=128, F_n=80, F_e=4, L=3, rrows=0, sa=4):
     out = {k: fwd[k] for k in ("node_tc", "edge_small", "edge_tc", "gate_tc", "readout_head",
                                "edge_gate_tc")}
     # forward with saves: the last layer also stores e' (edge kernels) and h (gather)
-    out["gather_segsum"] = fwd["gather_segsum"] + sa * N * d
+    # (+ the sign bits of h^0 .. h^{L-2}: the backward's LReLU' masks, d/8 bytes per node)
+    out["gather_segsum"] = fwd["gather_segsum"] + sa * N * d + (L - 1) * N * d // 8
     out["broadcast_dh"] = sa * N * d + s * N * d + 4 * N
     Ed, Nd = E * d, N * d
     out["gate_bwd"] = L * (sa * Ed + s * Nd + sa * Nd + 2 * s * Ed + 8 * E)
@@ -224,7 +225,7 @@ def train_algorithmic_bytes(N, E, B, d=128, F_n=80, F_e=4, L=3, rrows=0, sa=4):
     out["wgrad_tc"] = (L * (s * Ed + sa * Ed) + (L - 1) * (s * Ed + sa * Ed)
                        + (s * Nd + s * N * F_n) + (L - 1) * (s * Nd + sa * Nd))
     out["wgrad_skinny"] = s * Ed + s * E * F_e
-    out["dh_prev_tc"] = (L - 1) * (2 * s * Nd + sa * Nd)
+    out["dh_prev_tc"] = (L - 1) * (2 * s * Nd + Nd // 8)     # dP, dh^{i-1}, LReLU' sign bits
     out["split_reduce"] = 0
     return out
 

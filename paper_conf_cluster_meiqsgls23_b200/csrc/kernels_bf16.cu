@@ -611,7 +611,7 @@ int forward_layer_bf16(const occu_ctx *ctx, const DevCsr &csr, int layer, const 
     if ((r = launch_gather_segsoftmax_bf16(ctx, csr, a.g, a.hbar, a.h_out, a.rpart, a.save_w, st)) < 0) return r;
     return n + r;
   }
-  if ((r = launch_gather_segsum_bf16(ctx, csr, a.g, a.hbar, a.h_out, a.rpart, st)) < 0) return r;
+  if ((r = launch_gather_segsum_bf16(ctx, csr, a.g, a.hbar, a.h_out, a.rpart, st, a.h_bits)) < 0) return r;
   return n + r;
 }
 
@@ -678,7 +678,7 @@ static int forward_layer_bf16_256(const occu_ctx *ctx, const DevCsr &csr, int la
                               nullptr, nullptr, nullptr, "gate_tc", st)) < 0) return r;
     n += r;
   }
-  if ((r = launch_gather_segsum_bf16(ctx, csr, a.g, a.hbar, a.h_out, a.rpart, st)) < 0) return r;
+  if ((r = launch_gather_segsum_bf16(ctx, csr, a.g, a.hbar, a.h_out, a.rpart, st, a.h_bits)) < 0) return r;
   return n + r;
 }
 

@@ -615,7 +615,7 @@ __global__ void __launch_bounds__(NT, (BF ? G <= 8 : (G == 4 && !RP)) ? 4 : 3) g
     const int32_t *__restrict__ in_ptr, const int32_t *__restrict__ in_src, int N, int mean,
     float slope, void *__restrict__ h_out, const int32_t *__restrict__ node_graph,
     float *__restrict__ rpart, const float *__restrict__ hubsum = nullptr,
-    const int32_t *__restrict__ in_dst = nullptr) {
+    const int32_t *__restrict__ in_dst = nullptr, uint32_t *__restrict__ hbits = nullptr) {
   constexpr int V = D / 32;
   constexpr int NPW = 8;
   const int lane = threadIdx.x & 31;
@@ -659,6 +659,15 @@ __global__ void __launch_bounds__(NT, (BF ? G <= 8 : (G == 4 && !RP)) ? 4 : 3) g
         acc[c] = 0.f;
       }
       if (!RP || h_out) store_row_t<V, BF>(h_out, t0 + nd, D, lane, o);
+      if (hbits) {      // word c, bit l: channel V·l + c is positive (LReLU' = 1)
+        uint32_t mine = 0u;
+#pragma unroll
+        for (int c = 0; c < V; ++c) {
+          const uint32_t m = __ballot_sync(0xffffffffu, o[c] > 0.f);
+          if (lane == c) mine = m;
+        }
+        if (lane < V) hbits[(t0 + nd) * V + lane] = mine;
+      }
       if (RP) {
         const int gc = __shfl_sync(0xffffffffu, gr_l, nd);
         const int gn = __shfl_sync(0xffffffffu, gr_l, (nd + 1) & 31);
@@ -1989,7 +1998,7 @@ static int launch_hub_sums(const occu_ctx *ctx, const DevCsr &csr, const void *g
 
 template <int D>
 static int gather_impl(const occu_ctx *ctx, const DevCsr &csr, const float *g, const float *hbar,
-                       float *h_out, float *rpart, cudaStream_t st) {
+                       float *h_out, float *rpart, cudaStream_t st, uint32_t *hbits) {
   if (csr.N <= 0) return 0;
   static const int variant = [] {
     const char *e = getenv("OCCU_GATHER_V");
@@ -2004,7 +2013,8 @@ static int gather_impl(const occu_ctx *ctx, const DevCsr &csr, const float *g, c
   int r0 = launch_hub_sums<D, false>(ctx, csr, g, hbar, &hub, st);
   if (r0 < 0) return r0;
   OCCU_PROF_BEGIN(ctx, "gather_segsum", st);
-#define OCCU_GATHER_ARGS g, hbar, csr.in_ptr, csr.in_src, csr.N, mean, ctx->cfg.slope, h_out, csr.node_graph, rpart, hub, csr.in_dst
+#define OCCU_GATHER_ARGS g, hbar, csr.in_ptr, csr.in_src, csr.N, mean, ctx->cfg.slope, h_out, csr.node_graph, rpart, hub, csr.in_dst, hbits
+  if (hbits && variant != 1) return -int(cudaErrorInvalidValue);    // sign bits: default kernel only
   if constexpr (D == 256) {
     // d = 256: two (g, h̄) row pairs in flight per lane (16 floats each); 1 KB rows
     const int grid = grid_for(long(csr.N) * 4, NT, occ * ctx->num_sms);
@@ -2040,7 +2050,7 @@ static int gather_impl(const occu_ctx *ctx, const DevCsr &csr, const float *g, c
 
 template <int D>
 static int gather_bf16_impl(const occu_ctx *ctx, const DevCsr &csr, const void *g, const void *hbar,
-                            void *h_out, float *rpart, cudaStream_t st) {
+                            void *h_out, float *rpart, cudaStream_t st, uint32_t *hbits) {
   if (csr.N <= 0) return 0;
   const int mean = ctx->cfg.aggr == OCCU_AGGR_MEAN;
   static const int gsel = [] {
@@ -2056,7 +2066,7 @@ static int gather_bf16_impl(const occu_ctx *ctx, const DevCsr &csr, const void *
   int r0 = launch_hub_sums<D, true>(ctx, csr, g, hbar, &hub, st);
   if (r0 < 0) return r0;
   OCCU_PROF_BEGIN(ctx, "gather_segsum", st);
-#define OCCU_GB_ARGS g, hbar, csr.in_ptr, csr.in_src, csr.N, mean, ctx->cfg.slope, h_out, csr.node_graph, rpart, hub, csr.in_dst
+#define OCCU_GB_ARGS g, hbar, csr.in_ptr, csr.in_src, csr.N, mean, ctx->cfg.slope, h_out, csr.node_graph, rpart, hub, csr.in_dst, hbits
   if constexpr (D == 256) {
     if (rpart) launch_pdl(ctx->pdl & 64, gather_segsum_v2_kernel<D, 2, true, true>, grid, NT, 0, st, OCCU_GB_ARGS);
     else launch_pdl(ctx->pdl & 64, gather_segsum_v2_kernel<D, 2, false, true>, grid, NT, 0, st, OCCU_GB_ARGS);
@@ -2117,21 +2127,23 @@ int launch_gather_segsoftmax_bf16(const occu_ctx *ctx, const DevCsr &csr, void *
 }
 
 int launch_gather_segsum_bf16(const occu_ctx *ctx, const DevCsr &csr, const void *g,
-                              const void *hbar, void *h_out, float *rpart, cudaStream_t st) {
+                              const void *hbar, void *h_out, float *rpart, cudaStream_t st,
+                              uint32_t *h_bits) {
   switch (ctx->cfg.d) {
-    case 64: return gather_bf16_impl<64>(ctx, csr, g, hbar, h_out, rpart, st);
-    case 128: return gather_bf16_impl<128>(ctx, csr, g, hbar, h_out, rpart, st);
-    case 256: return gather_bf16_impl<256>(ctx, csr, g, hbar, h_out, rpart, st);
+    case 64: return gather_bf16_impl<64>(ctx, csr, g, hbar, h_out, rpart, st, h_bits);
+    case 128: return gather_bf16_impl<128>(ctx, csr, g, hbar, h_out, rpart, st, h_bits);
+    case 256: return gather_bf16_impl<256>(ctx, csr, g, hbar, h_out, rpart, st, h_bits);
     default: return -int(cudaErrorInvalidValue);
   }
 }
 
 int launch_gather_segsum(const occu_ctx *ctx, const DevCsr &csr, const float *g,
-                         const float *hbar, float *h_out, float *rpart, cudaStream_t st) {
+                         const float *hbar, float *h_out, float *rpart, cudaStream_t st,
+                         uint32_t *h_bits) {
   switch (ctx->cfg.d) {
-    case 64: return gather_impl<64>(ctx, csr, g, hbar, h_out, rpart, st);
-    case 128: return gather_impl<128>(ctx, csr, g, hbar, h_out, rpart, st);
-    case 256: return gather_impl<256>(ctx, csr, g, hbar, h_out, rpart, st);
+    case 64: return gather_impl<64>(ctx, csr, g, hbar, h_out, rpart, st, h_bits);
+    case 128: return gather_impl<128>(ctx, csr, g, hbar, h_out, rpart, st, h_bits);
+    case 256: return gather_impl<256>(ctx, csr, g, hbar, h_out, rpart, st, h_bits);
     default: return -int(cudaErrorInvalidValue);
   }
 }
@@ -2335,6 +2347,7 @@ static int backward_layer_impl(occu_ctx *ctx, const DevCsr &csr, const BwdLayerA
   if (w.partial.ensure(3 * WG_SLOT_FLOATS * 4) != cudaSuccess) return -int(cudaErrorMemoryAllocation);
   float *slot = w.partial.as<float>();
   static const bool fuse_we = !getenv("OCCU_NO_FUSE_WE");   // A/B switch: dW_e in the layer-1 edge backward
+  static const bool use_bits = !getenv("OCCU_NO_HBITS");     // A/B switch: LReLU'(h_in) from the sign bits
   int we_blocks = 0;                        // > 0: dW_e partials already written by edge_bwd_small
   // the streaming gate backward (saved gates) leaves MG = dA[t] ⊙ g to the node backward
   const bool mg_from_g = tc && a.g && !getenv("OCCU_NODE_BWD_V1");
@@ -2477,7 +2490,8 @@ static int backward_layer_impl(occu_ctx *ctx, const DevCsr &csr, const BwdLayerA
   n += r;
   if (a.dh_prev && csr.N > 0 && tc) {   // dh^{i-1} = dP W_u on tensor cores
     if ((r = launch_plain_tc(ctx, w.dP.as<float>(), D, csr.N, 5, i, nullptr, a.dh_prev,
-                             "dh_prev_tc", st, a.h_in, csr.in_ptr, in_bf)) < 0) return r;
+                             "dh_prev_tc", st, a.h_in, csr.in_ptr, in_bf,
+                             use_bits ? a.h_in_bits : nullptr)) < 0) return r;
     n += r;
   } else if (a.dh_prev && csr.N > 0) {   // dh^{i-1} = dP W_u  (K == D for i > 0)
     const size_t sm1 = (size_t(D) * D + BM * (D + 4)) * 4;

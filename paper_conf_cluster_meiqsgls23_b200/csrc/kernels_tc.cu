@@ -122,6 +122,8 @@ struct RowGemmArgs {
   const float *dh, *h, *hbar, *e, *de;
   const float *mask_h;     // PLAIN: multiply row by LReLU'(mask_h row) (÷ deg for MEAN) -> dA
   int mask_bf;             // mask_h rows are BF16 (OCCU_BF16 training)
+  const uint32_t *mask_bits;   // PLAIN: the mask's sign bits [R][D/32] (word c, bit l: channel V·l + c)
+                               // instead of mask_h rows (gather_segsum's training output)
   const float *bias;       // PLAIN: per-column bias (nullable), then ReLU if relu
   int relu;
   const int32_t *in_ptr;
@@ -451,7 +453,15 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
       // stream of the de / dh_prev GEMMs — one chunk ahead
       float4 dpre[4];
       const float *pre_src = EPI == EPI_EDGEBWD ? a.de
-                           : (EPI == EPI_PLAIN ? (a.add ? a.add : (a.mask_bf ? nullptr : a.mask_h)) : nullptr);
+                           : (EPI == EPI_PLAIN ? (a.add ? a.add : ((a.mask_bf || a.mask_bits) ? nullptr : a.mask_h)) : nullptr);
+      // PLAIN with sign bits: the row's D/32 mask words (16 B at D = 128) instead of a D-float row
+      constexpr int MV = D / 32;
+      uint32_t mw[EPI == EPI_PLAIN ? MV : 1];
+      if (EPI == EPI_PLAIN) {
+#pragma unroll
+        for (int c = 0; c < (EPI == EPI_PLAIN ? MV : 1); ++c)
+          mw[c] = (a.mask_bits && live) ? __ldg(a.mask_bits + (r0 + row) * MV + c) : 0u;
+      }
       if (EPI == EPI_EDGEBWD || EPI == EPI_PLAIN) {
 #pragma unroll
         for (int u = 0; u < 4; ++u)
@@ -494,7 +504,19 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
           float o[16];
 #pragma unroll
           for (int u = 0; u < 16; ++u) o[u] = __uint_as_float(r[u]) * un;
-          if (a.mask_h && live) {
+          if (a.mask_bits && live) {
+            float dsc = 1.f;
+            if (a.mean) {
+              const int deg = __ldg(a.in_ptr + grow + 1) - __ldg(a.in_ptr + grow);
+              dsc = float(deg > 0 ? deg : 1);
+            }
+            const int sh = (cb + c0) / MV;                 // cb + c0 is a multiple of 16 (and of MV)
+#pragma unroll
+            for (int u = 0; u < 16; ++u) {
+              o[u] *= ((mw[u % MV] >> (sh + u / MV)) & 1u) ? 1.f : a.slope;
+              if (a.mean) o[u] = o[u] / dsc;
+            }
+          } else if (a.mask_h && live) {
             const float *mr = a.mask_h + grow * D + cb + c0;
             const uint16_t *mb = reinterpret_cast<const uint16_t *>(a.mask_h) + grow * D + cb + c0;
             float dsc = 1.f;
@@ -2454,7 +2476,7 @@ static int tc_forward_layer_pair(const occu_ctx *ctx, const DevCsr &csr, int lay
     if ((r = launch_rowgemm_pair<EPI_GATE, false, true>(ctx, rg, "gate_tc", st)) < 0) return r;
     n += r;
   }
-  if ((r = launch_gather_segsum(ctx, csr, a.g, a.hbar, a.h_out, a.rpart, st)) < 0) return r;
+  if ((r = launch_gather_segsum(ctx, csr, a.g, a.hbar, a.h_out, a.rpart, st, a.h_bits)) < 0) return r;
   return n + r;
 }
 
@@ -2588,7 +2610,7 @@ static int tc_forward_layer_impl(const occu_ctx *ctx, const DevCsr &csr, int lay
     n += r;
   } else {
     // a5 + a6: gather + segmented sum (CUDA cores, warp per 8 destinations)
-    if ((r = launch_gather_segsum(ctx, csr, a.g, a.hbar, a.h_out, a.rpart, st)) < 0) return r;
+    if ((r = launch_gather_segsum(ctx, csr, a.g, a.hbar, a.h_out, a.rpart, st, a.h_bits)) < 0) return r;
     n += r;
   }
   return n;
@@ -2610,9 +2632,10 @@ static int bwd_gate_impl(const occu_ctx *ctx, const DevCsr &csr, int layer, cons
 template <int D>
 static int plain_impl(const occu_ctx *ctx, const float *A, int K, int R, int wkind, int layer,
                       const float *add, float *out, const char *name, cudaStream_t st,
-                      const float *mask_h, const int32_t *in_ptr, bool mask_bf) {
+                      const float *mask_h, const int32_t *in_ptr, bool mask_bf, const uint32_t *mask_bits) {
   RowGemmArgs r{};
   r.mask_bf = mask_bf ? 1 : 0;
+  r.mask_bits = mask_bits;
   r.slope = ctx->cfg.slope;
   r.A = A; r.K = K; r.R = R; r.add = add; r.out = out;
   r.wimg = tc_wimg(ctx, wkind, layer); r.wfexp = tc_wfexp(ctx, wkind, layer);
@@ -2670,10 +2693,10 @@ int launch_bwd_gate_tc(const occu_ctx *ctx, const DevCsr &csr, int layer, const 
 }
 int launch_plain_tc(const occu_ctx *ctx, const float *A, int K, int R, int wkind, int layer,
                     const float *add, float *out, const char *name, cudaStream_t st,
-                    const float *mask_h, const int32_t *in_ptr, bool mask_bf) {
+                    const float *mask_h, const int32_t *in_ptr, bool mask_bf, const uint32_t *mask_bits) {
   if (R <= 0) return 0;
-  return ctx->cfg.d == 64 ? plain_impl<64>(ctx, A, K, R, wkind, layer, add, out, name, st, mask_h, in_ptr, mask_bf)
-                          : plain_impl<128>(ctx, A, K, R, wkind, layer, add, out, name, st, mask_h, in_ptr, mask_bf);
+  return ctx->cfg.d == 64 ? plain_impl<64>(ctx, A, K, R, wkind, layer, add, out, name, st, mask_h, in_ptr, mask_bf, mask_bits)
+                          : plain_impl<128>(ctx, A, K, R, wkind, layer, add, out, name, st, mask_h, in_ptr, mask_bf, mask_bits);
 }
 int launch_bias_tc(const occu_ctx *ctx, const float *A, int K, int R, int wkind, int layer,
                    const float *bias, bool relu, float *out, const char *name, cudaStream_t st) {

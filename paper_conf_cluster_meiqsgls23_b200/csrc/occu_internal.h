@@ -78,6 +78,7 @@ struct Workspace {
   DevBuf gdh[2];           // training: gradients w.r.t. the stack's node states (ping-pong)
   DevBuf dbwd;             // training: decoder backward rows / stats / partials
   DevBuf hub;              // aggregation: per-64-edge-unit partials of hub segments
+  std::vector<DevBuf> hbits;   // training: per layer sign bitmask of h [N][d/32] (LReLU' masks)
   void release_all();
 };
 
@@ -136,6 +137,7 @@ struct occu_ctx {
   bool have_forward = false;
   bool h_last_stored = true;   // false: the last forward kept only readout partials of h_L
   bool small_fwd = false;      // the last forward ran the single-CTA small-batch kernel
+  int hbits_layers = 0;        // the last forward wrote the sign bits of h^0 .. h^{hbits_layers-1}
   bool small_enabled = true;   // occu_set_small_batch_kernel: single-CTA forward for tiny batches (default on)
   int64_t launches = 0;
   mutable occu::Profiler prof;
@@ -197,6 +199,7 @@ struct FwdLayerArgs {
   // then be null).  See gather_segsum_kernel / readout_head_kernel.
   const int32_t *e_eid; float *e0_out; float *rpart;
   bool save_w = false;                 // reading B, training: g receives the softmax weights
+  uint32_t *h_bits = nullptr;          // training: sign bitmask of h_out for the backward's LReLU'
 };
 int launch_forward_layer(const occu_ctx *ctx, const DevCsr &csr, const FwdLayerArgs &a,
                          cudaStream_t st);
@@ -212,7 +215,7 @@ int launch_bwd_gate_tc(const occu_ctx *ctx, const DevCsr &csr, int layer, const 
 int launch_plain_tc(const occu_ctx *ctx, const float *A, int K, int R, int wkind, int layer,
                     const float *add, float *out, const char *name, cudaStream_t st,
                     const float *mask_h = nullptr, const int32_t *in_ptr = nullptr,
-                    bool mask_bf = false);
+                    bool mask_bf = false, const uint32_t *mask_bits = nullptr);
 // OCCU_BF16 training: z = W_e e_in recomputed from BF16 e_in on the BF16 tensor-core path
 // (as the forward), epilogue dy = de ⊙ e' ⊙ σ(-αz) with BF16 e', dα = <dy, z>, DZ = α dy.
 int launch_bwd_edge_bf16(const occu_ctx *ctx, const DevCsr &csr, int layer, const void *e_in,
@@ -227,7 +230,8 @@ size_t tc_partial_floats(int E, int D);
 int launch_forward_layer_tc(const occu_ctx *ctx, const DevCsr &csr, int layer, const FwdLayerArgs &a,
                             float *partial, cudaStream_t st);
 int launch_gather_segsum(const occu_ctx *ctx, const DevCsr &csr, const float *g,
-                         const float *hbar, float *h_out, float *rpart, cudaStream_t st);
+                         const float *hbar, float *h_out, float *rpart, cudaStream_t st,
+                         uint32_t *h_bits = nullptr);
 // Reading B (OCCU_MSG_NEIGHBOR_SOFTMAX, NEXT-1): v holds the logits W_m e'; the per-channel
 // softmax over each destination's in-edges, the message product and the segmented sum in one
 // pass; write_w (training) overwrites v with the softmax weights for the backward.
@@ -237,7 +241,8 @@ int launch_gather_segsoftmax(const occu_ctx *ctx, const DevCsr &csr, float *v, c
 int launch_gather_segsoftmax_bf16(const occu_ctx *ctx, const DevCsr &csr, void *v, const void *hbar,
                                   void *h_out, float *rpart, bool write_w, cudaStream_t st);
 int launch_gather_segsum_bf16(const occu_ctx *ctx, const DevCsr &csr, const void *g,
-                              const void *hbar, void *h_out, float *rpart, cudaStream_t st);
+                              const void *hbar, void *h_out, float *rpart, cudaStream_t st,
+                              uint32_t *h_bits = nullptr);
 // OCCU_BF16 forward layer (kernels_bf16.cu); FwdLayerArgs pointers to h̄, e', g, h hold BF16.
 int launch_pair_bf16(const occu_ctx *ctx, int epi, bool af32, const void *A, int K, int R, int layer,
                      void *out, const float *a_s, const float *a_d, float *p, float *q,
@@ -309,6 +314,8 @@ struct BwdLayerArgs {
   const float *de_out;                // [E][d] gradient w.r.t. e^i from layer i+1 (nullable)
   float *de_prev;                     // [E][Ke] (nullable at layer 0)
   float *dh_prev;                     // [N][K]  (nullable at layer 0)
+  const uint32_t *h_in_bits = nullptr;  // sign bitmask of h_in (gather_segsum, training forward):
+                                      // LReLU'(h^{i-1}) for dh_prev without re-reading h_in rows
   bool bf = false;                    // OCCU_BF16: hbar, e, g, h and (layer > 0) h_in, e_in
                                       // point to BF16 rows; gradients stay FP32 (R28)
 };

@@ -53,7 +53,7 @@ void Workspace::release_all() {
                     &aef[0], &aef[1], &acsr[0], &acsr[1], &dT, &dZ, &dprep, &dpool, &gx, &gqkv, &go, &gscr, &gdh[0], &gdh[1], &dbwd, &hub, &aty[0], &aty[1], &rowexp,
                     &scsr, &snf, &sef, &sdesc, &hf};
   for (DevBuf *b : bufs) b->release();
-  for (auto *v : {&hbar, &p, &q, &e, &h, &gs, &gh, &gsave})
+  for (auto *v : {&hbar, &p, &q, &e, &h, &gs, &gh, &gsave, &hbits})
     for (DevBuf &b : *v) b.release();
 }
 
@@ -263,6 +263,7 @@ occu_status forward(occu_ctx *ctx, const DevCsr &csr, const float *nf, const flo
   if (st != OCCU_OK) return st;
   cudaStream_t s = ctx->stream;
   const float *P = ctx->params.as<float>();
+  ctx->hbits_layers = 0;
   const bool bf = c.prec == OCCU_BF16;        // kernel path 0 only (occu_set_kernel_path)
   const bool tc = bf || (ctx->path != 1 && tc_supported(c));
   if (!save_all && ctx->path == 0 && ctx->small_enabled && small_forward_ok(ctx, csr)) {
@@ -314,6 +315,13 @@ occu_status forward(occu_ctx *ctx, const DevCsr &csr, const float *nf, const flo
     }
     a.h_out = w.h[i].as<float>();
     a.save_w = save_all && c.msg == OCCU_MSG_NEIGHBOR_SOFTMAX;   // reading B: weights for the backward
+    if (save_all && tc && ctx->path == 0 && !last && c.msg == OCCU_MSG_CHANNEL_SOFTMAX) {
+      // sign bits of h^i: the backward's LReLU'(h^i) mask of dh^i (dh_prev of layer i+1)
+      if (w.hbits.size() < size_t(c.L)) w.hbits.resize(c.L);
+      CK(w.hbits[i].ensure(size_t(csr.N) * (c.d / 32) * 4), "alloc h sign bits");
+      a.h_bits = reinterpret_cast<uint32_t *>(w.hbits[i].ptr);
+      ctx->hbits_layers = i + 1;
+    }
     if (tc) {
       a.e_out = w.e[i].as<float>();            // the gate kernel re-reads e'
       if (last && fuse_ro) {
@@ -505,6 +513,7 @@ occu_status grads_core(occu_ctx *ctx, const DevCsr &csr, const Staged &stg, int3
     a.de_out = i < c.L - 1 ? w.deB.as<float>() : nullptr;
     a.de_prev = i > 0 ? w.deB.as<float>() : nullptr;     // read-before-write ordering, see DESIGN
     a.dh_prev = i > 0 ? w.dh.as<float>() : nullptr;
+    if (i > 0 && ctx->hbits_layers >= i) a.h_in_bits = reinterpret_cast<const uint32_t *>(w.hbits[i - 1].ptr);
     a.bf = c.prec == OCCU_BF16;     // h̄, e', g, h (and h_in, e_in for i > 0) stored as BF16
     LK(launch_backward_layer(ctx, csr, a, s), "backward layer");
   }
