@@ -210,9 +210,9 @@ def train_algorithmic_bytes(N, E, B, d=128, F_n=80, F_e=4, L=3, rrows=0, sa=4):
     out = {k: fwd[k] for k in ("node_tc", "edge_small", "edge_tc", "gate_tc", "readout_head",
                                "edge_gate_tc")}
     # forward with saves: the last layer also stores e' (edge kernels) and h (gather)
-    # (+ the sign bits of h^0 .. h^{L-2}: the backward's LReLU' masks, d/8 bytes per node)
-    out["gather_segsum"] = fwd["gather_segsum"] + sa * N * d + (L - 1) * N * d // 8
-    out["broadcast_dh"] = sa * N * d + s * N * d + 4 * N
+    # (+ the sign bits of h^0 .. h^{L-1}: the backward's LReLU' masks, d/8 bytes per node)
+    out["gather_segsum"] = fwd["gather_segsum"] + sa * N * d + L * N * d // 8
+    out["broadcast_dh"] = N * d // 8 + s * N * d + 4 * N      # h_L's sign bits, dh
     Ed, Nd = E * d, N * d
     out["gate_bwd"] = L * (sa * Ed + s * Nd + sa * Nd + 2 * s * Ed + 8 * E)
     out["de_tc"] = L * (2 * s * Ed) + (L - 1) * s * Ed

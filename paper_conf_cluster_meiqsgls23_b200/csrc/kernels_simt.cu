@@ -1291,7 +1291,10 @@ __global__ void broadcast_dh_kernel(const float *__restrict__ dr, const int32_t 
                                     const int32_t *__restrict__ node_off, int N, int D,
                                     const void *__restrict__ h_mask, int mask_bf,
                                     const int32_t *__restrict__ in_ptr,
-                                    int mean, float slope, float *__restrict__ dh) {
+                                    int mean, float slope, float *__restrict__ dh,
+                                    const uint32_t *__restrict__ h_bits) {
+  // h_bits (training forward's sign bits of h_L, word c / bit l = channel V·l + c) replace the
+  // h_L rows as the LReLU' mask: D/8 bytes per node instead of a D-wide row
   const int D4 = D / 4;
   const long total = long(N) * D4;
   for (long i = blockIdx.x * long(blockDim.x) + threadIdx.x; i < total;
@@ -1301,9 +1304,22 @@ __global__ void broadcast_dh_kernel(const float *__restrict__ dr, const int32_t 
     const float inv = 1.f / float(__ldg(node_off + b + 1) - __ldg(node_off + b));
     const float4 r = __ldg(reinterpret_cast<const float4 *>(dr + long(b) * D) + k4);
     float v[4] = {r.x * inv, r.y * inv, r.z * inv, r.w * inv};
-    if (h_mask) {
+    if (h_bits || h_mask) {
       float hm[4];
-      if (mask_bf) {
+      if (h_bits && D == 128) {        // channel 4·k4 + c: word c, bit k4
+        const uint4 w = __ldg(reinterpret_cast<const uint4 *>(h_bits) + u);
+        hm[0] = (w.x >> k4) & 1u ? 1.f : -1.f;
+        hm[1] = (w.y >> k4) & 1u ? 1.f : -1.f;
+        hm[2] = (w.z >> k4) & 1u ? 1.f : -1.f;
+        hm[3] = (w.w >> k4) & 1u ? 1.f : -1.f;
+      } else if (h_bits) {
+        const int V = D / 32;
+#pragma unroll
+        for (int c = 0; c < 4; ++c) {
+          const int ch = 4 * k4 + c;
+          hm[c] = (__ldg(h_bits + long(u) * V + ch % V) >> (ch / V)) & 1u ? 1.f : -1.f;
+        }
+      } else if (mask_bf) {
         const uint2 x = __ldg(reinterpret_cast<const uint2 *>(reinterpret_cast<const uint16_t *>(h_mask) + long(u) * D) + k4);
         hm[0] = __uint_as_float(x.x << 16); hm[1] = __uint_as_float(x.x & 0xFFFF0000u);
         hm[2] = __uint_as_float(x.y << 16); hm[3] = __uint_as_float(x.y & 0xFFFF0000u);
@@ -2291,6 +2307,7 @@ int launch_wgrad(occu_ctx *ctx, const float *X, int A, const void *Y, int Bn, lo
 
 int launch_head_backward(occu_ctx *ctx, const DevCsr &csr, const float *targets, int global_B,
                          cudaStream_t st) {
+  static const bool use_bits = !getenv("OCCU_NO_HBITS");
   const occu_config &cf = ctx->cfg;
   const ParamLayout &L = ctx->layout;
   Workspace &w = ctx->ws;
@@ -2321,7 +2338,8 @@ int launch_head_backward(occu_ctx *ctx, const DevCsr &csr, const float *targets,
       w.dr.as<float>(), csr.node_graph, csr.node_off, csr.N, cf.d,
       tcb ? w.h[cf.L - 1].ptr : nullptr, cf.prec == OCCU_BF16 ? 1 : 0, csr.in_ptr,
       cf.aggr == OCCU_AGGR_MEAN, cf.slope,
-      w.dh.as<float>());
+      w.dh.as<float>(), (tcb && use_bits && ctx->hbits_layers >= cf.L)
+                            ? reinterpret_cast<const uint32_t *>(w.hbits[cf.L - 1].ptr) : nullptr);
   OCCU_PROF_END(ctx);
   LAUNCH_CHECK();
   return 3;

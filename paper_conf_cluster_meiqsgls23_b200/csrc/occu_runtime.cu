@@ -315,8 +315,9 @@ occu_status forward(occu_ctx *ctx, const DevCsr &csr, const float *nf, const flo
     }
     a.h_out = w.h[i].as<float>();
     a.save_w = save_all && c.msg == OCCU_MSG_NEIGHBOR_SOFTMAX;   // reading B: weights for the backward
-    if (save_all && tc && ctx->path == 0 && !last && c.msg == OCCU_MSG_CHANNEL_SOFTMAX) {
-      // sign bits of h^i: the backward's LReLU'(h^i) mask of dh^i (dh_prev of layer i+1)
+    if (save_all && tc && ctx->path == 0 && c.msg == OCCU_MSG_CHANNEL_SOFTMAX) {
+      // sign bits of h^i: the backward's LReLU'(h^i) mask of dh^i (dh_prev of layer i+1; the
+      // head backward's broadcast for i = L-1)
       if (w.hbits.size() < size_t(c.L)) w.hbits.resize(c.L);
       CK(w.hbits[i].ensure(size_t(csr.N) * (c.d / 32) * 4), "alloc h sign bits");
       a.h_bits = reinterpret_cast<uint32_t *>(w.hbits[i].ptr);
