@@ -132,6 +132,7 @@ struct RowGemmArgs {
   float *part;             // GATEAGG: [R/32 units][2 slots][D] boundary-segment partials
   int rev;                 // walk tiles last-to-first (reads what the previous kernel wrote last, still in L2)
   const int *rexp;         // d = 256 NODE: per-row scale exponents (row_exp_kernel)
+  int dot2;                // EDGEBWD: dα by the compensated FP32 dot (else float64 FMA)
 };
 
 struct Smem {
@@ -561,7 +562,11 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
           warp_store_chunk<D>(wbuf, a.out, wrow0, wrows, cb + c0, o, lane);
         }
       } else if (EPI == EPI_EDGEBWD) {
-        double dpart = 0.0;                          // dα = <dy, z> in float64 (cancellation)
+        // dα = <dy, z> needs more than FP32 (cancellation): compensated FP32 dot (Ogita-Rump-
+        // Oishi Dot2: TwoProduct by FMA + TwoSum, as accurate as a 2x-precision sum rounded
+        // once) — 9 FP32 operations per element instead of two F2F.F64 conversions and a DFMA
+        double dpart = 0.0;
+        float ds = 0.f, dc = 0.f;
 #pragma unroll 1
         for (int c0 = 0; c0 < DH; c0 += 16) {
           uint32_t r[16];
@@ -602,13 +607,22 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
               const float z = __uint_as_float(r[u + t]) * un;
               // σ'(y) = σ(y)·σ(-y), y = α z (recomputed): no 1 - e' cancellation
               const float dy = dvv[t] * evv[t] * sneg[t];
-              dpart = fma(double(dy), double(z), dpart);
+              if (a.dot2) {
+                const float pr = dy * z, pe = fmaf(dy, z, -pr);          // TwoProduct
+                const float t1 = ds + pr, bp = t1 - ds;                  // TwoSum(ds, pr)
+                const float se = (ds - (t1 - bp)) + (pr - bp);
+                ds = t1;
+                dc += se + pe;
+              } else {
+                dpart = fma(double(dy), double(z), dpart);
+              }
               o[u + t] = aux * dy;
             }
           }
           warp_store_chunk<D>(wbuf, a.out, wrow0, wrows, cb + c0, o, lane);
         }
         double *xd = reinterpret_cast<double *>(xg);   // reuses the whole exchange area
+        if (a.dot2) dpart = double(ds) + double(dc);
         group_bar(g);                                   // everyone has consumed the α slot
         xd[hf * 128 + row] = dpart;
         group_bar(g);
@@ -2371,8 +2385,14 @@ static int launch_rowgemm(const occu_ctx *ctx, const RowGemmArgs &ra, const char
   const int grid = std::min(tiles, ctx->num_sms);
   CUtensorMap tmap;
   if (!encode_rows_map(&tmap, ra.A, ra.R, ra.K)) return -int(cudaErrorInvalidValue);
+  static const int dot2 = [] {
+    const char *e = getenv("OCCU_DA_F64");
+    return e && atoi(e) ? 0 : 1;
+  }();
+  RowGemmArgs rc = ra;
+  rc.dot2 = dot2;
   OCCU_PROF_BEGIN(ctx, name, st);
-  launch_pdl(ctx->pdl & 1, rowgemm_kernel<D, EPI>, grid, NTH, smem, st, tmap, ra);
+  launch_pdl(ctx->pdl & 1, rowgemm_kernel<D, EPI>, grid, NTH, smem, st, tmap, rc);
   OCCU_PROF_END(ctx);
   TC_CHECK();
   return 1;
