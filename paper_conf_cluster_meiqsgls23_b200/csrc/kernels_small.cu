@@ -10,11 +10,12 @@
 // The three row-GEMMs of a layer run on the tensor cores through mma.sync m16n8k8 TF32 with
 // the 3xTF32 split (x = hi + lo, hi = x with its low 13 mantissa bits cleared: products
 // lo·hi + hi·lo + hi·hi accumulated in FP32, ~2^-20 relative — FP32-accurate for the 1e-4
-// contract), one warp per 16 rows x all D output channels (m16n8k8 measured at 512 MAC/cycle
+// contract), four warps per 16 rows x D output channels (m16n8k8 measured at 512 MAC/cycle
 // on one SM, 4x the FP32 FMA rate; the SIMT register-blocked version was bound by shared-memory
 // wavefronts).  The step that follows each GEMM runs in its epilogue from the accumulator
 // fragments — LeakyReLU and the p = h̄·a_s, q = h̄·a_d dots (a2), σ(α z) (a3), the channel
-// softmax (a4) — with the row reductions as xor-shuffles over the 4 lanes that share a row.
+// softmax (a4) — with the row reductions as xor-shuffles over the 4 lanes that share a row
+// and a fixed-order combination of the tile's 4 warps through shared memory.
 // Activation rows are padded to a stride that is an odd multiple of 4 words, so the fragment
 // loads (8 rows x 4 consecutive k) are conflict-free.  The a1 permutation is folded into the
 // layer-1 edge GEMM's row map (edge features staged in input order).
@@ -32,6 +33,7 @@ namespace {
 constexpr int SNMAX = 64, SEMAX = 128, SKMAX = 128, ST = 512;
 constexpr size_t SMEM_MAX = 220 * 1024;
 constexpr float LOG2E_S = 1.4426950408889634f;
+constexpr int XR_FLOATS = (ST / 32 / 4) * 4 * 16 * 2;
 
 struct SmallArgs {
   const float *nf, *ef;                      // [N][F_n], [E][F_e] (input edge order)
@@ -74,19 +76,25 @@ __device__ __forceinline__ void cpa_commit() { asm volatile("cp.async.commit_gro
 template <int N>
 __device__ __forceinline__ void cpa_wait() { asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory"); }
 
-// rows x cols floats (global row stride gld, shared row stride sld; cols % 4 == 0): warp per
-// row, lanes over 16-byte chunks — no integer division, and one out-of-line copy of the code
-// (the kernel body must stay small: it runs once per launch on one SM, so every instruction
-// is fetched cold from L2 once the body outgrows the 32 KB L1.5 instruction cache)
+// rows x cols floats (global row stride gld, shared row stride sld; cols % 4 == 0): 16-byte
+// chunks flattened over all threads (row = chunk / (cols/4) by a multiply-high with a
+// precomputed reciprocal: exact for the < 2^16 chunks of a staging call), one out-of-line copy
+// of the code (the kernel body must stay small: it runs once per launch on one SM, so every
+// instruction is fetched cold from L2 once the body outgrows the 32 KB L1.5 instruction cache)
 __device__ __noinline__ void stage_rows(float *dst, int sld, const float *__restrict__ src, int gld,
                                         int rows, int cols) {
-  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   if ((reinterpret_cast<uintptr_t>(src) & 15) == 0 && gld % 4 == 0 && sld % 4 == 0) {
-    for (int n = warp; n < rows; n += ST / 32)
-      for (int k = 4 * lane; k < cols; k += 128) cpa16(dst + n * sld + k, src + long(n) * gld + k);
+    const uint32_t c4 = uint32_t(cols) / 4, magic = 0xFFFFFFFFu / c4 + 1u;
+    for (uint32_t i = threadIdx.x; i < uint32_t(rows) * c4; i += ST) {
+      const uint32_t n = __umulhi(i, magic), k = 4u * (i - n * c4);
+      cpa16(dst + n * sld + k, src + long(n) * gld + k);
+    }
   } else {
-    for (int n = warp; n < rows; n += ST / 32)
-      for (int k = lane; k < cols; k += 32) cpa4(dst + n * sld + k, src + long(n) * gld + k);
+    const uint32_t magic = 0xFFFFFFFFu / uint32_t(cols) + 1u;
+    for (uint32_t i = threadIdx.x; i < uint32_t(rows) * uint32_t(cols); i += ST) {
+      const uint32_t n = __umulhi(i, magic), k = i - n * uint32_t(cols);
+      cpa4(dst + n * sld + k, src + long(n) * gld + k);
+    }
   }
 }
 
@@ -103,6 +111,7 @@ struct GemmEpi {
   const float *av;          // [2][D] a_s, a_d of the layer (G_NODE)
   float *pq;                // [2][SNMAX] p, q (written by G_NODE, read by G_EDGE)
   const int32_t *isrc, *idst;
+  float *xr;                // [ST/32/4 tile slots][4 warps][16 rows][2] row-partial exchange
 };
 
 __device__ __forceinline__ void split_tf32(float x, uint32_t &hi, uint32_t &lo) {
@@ -117,23 +126,30 @@ __device__ __forceinline__ void mma_tf32(float (&c)[4], const uint32_t (&a)[4], 
 }
 
 // Y[r][n] = epi(Σ_k X[xrow(r)][k] Ws[n][k]) for r < R, n < D (row stride ldy; Ws row stride
-// K + 4).  Warp = m-tile of 16 rows, all D/8 n-tiles; fragment lane (g, t) = (lane/4, lane%4)
-// holds rows g, g+8, and output columns 8nt + 2t, 8nt + 2t + 1 of every n-tile.
+// K + 4).  An m-tile of 16 rows is shared by WPT = 4 consecutive warps, warp q of the tile owning
+// n-tiles [q·NTW, (q+1)·NTW) (NTW = D/32); fragment lane (g, t) = (lane/4, lane%4) holds rows
+// g, g+8 and columns 8nt + 2t, 8nt + 2t + 1 of its n-tiles.  Row reductions (p, q dots, softmax
+// max / sum) combine the 4 warps' partials through shared memory (xr) in warp order, behind a
+// named barrier of the tile's 128 threads.
+constexpr int WPT = 4;
 template <int D, int EPI>
 __device__ __forceinline__ void tgemm(const float *X, int ldx, const int32_t *xmap, int R, int K,
                                       const float *Ws, float *Y, int ldy, const GemmEpi &ep) {
-  constexpr int NT = D / 8;
+  constexpr int NTW = D / 8 / WPT;
   const int lane = threadIdx.x & 31, g = lane >> 2, tq = lane & 3;
   const int MT = (R + 15) >> 4, ldw = K + 4;
-  for (int mt = threadIdx.x >> 5; mt < MT; mt += ST / 32) {
+  for (int wu = threadIdx.x >> 5; wu < MT * WPT; wu += ST / 32) {
+    const int mt = wu / WPT, ns = wu % WPT, slot = mt % (ST / 32 / WPT);
+    const int bar = 1 + slot;                    // named barrier of the tile's 4 warps
+    float *xs = ep.xr + slot * (WPT * 16 * 2);   // [WPT warps][16 rows][2 values]
     const int ra = mt * 16 + g, rb = ra + 8;
     const bool va = ra < R, vb = rb < R;
     const int ia = min(ra, R - 1), ib = min(rb, R - 1);
     const float *xa = X + (xmap ? xmap[ia] : ia) * ldx, *xb = X + (xmap ? xmap[ib] : ib) * ldx;
-    float c[NT][4];
+    float c[NTW][4];
 #pragma unroll
-    for (int nt = 0; nt < NT; ++nt) c[nt][0] = c[nt][1] = c[nt][2] = c[nt][3] = 0.f;
-#pragma unroll 1
+    for (int nt = 0; nt < NTW; ++nt) c[nt][0] = c[nt][1] = c[nt][2] = c[nt][3] = 0.f;
+#pragma unroll 2
     for (int k0 = 0; k0 < K; k0 += 8) {
       const int k1 = k0 + tq, k2 = k1 + 4;
       const bool m1 = k1 < K, m2 = k2 < K;
@@ -143,8 +159,8 @@ __device__ __forceinline__ void tgemm(const float *X, int ldx, const int32_t *xm
       split_tf32(m2 ? xa[k2] : 0.f, ah[2], al[2]);
       split_tf32(m2 ? xb[k2] : 0.f, ah[3], al[3]);
 #pragma unroll
-      for (int nt = 0; nt < NT; ++nt) {
-        const float *w = Ws + (nt * 8 + g) * ldw;
+      for (int nt = 0; nt < NTW; ++nt) {
+        const float *w = Ws + ((ns * NTW + nt) * 8 + g) * ldw;
         uint32_t bh0, bl0, bh1, bl1;
         split_tf32(m1 ? w[k1] : 0.f, bh0, bl0);
         split_tf32(m2 ? w[k2] : 0.f, bh1, bl1);
@@ -153,14 +169,32 @@ __device__ __forceinline__ void tgemm(const float *X, int ldx, const int32_t *xm
         mma_tf32(c[nt], ah, bh0, bh1);
       }
     }
+    auto tile_bar = [&]() { asm volatile("bar.sync %0, %1;" ::"r"(bar), "r"(WPT * 32) : "memory"); };
+    // row totals over the tile's 4 warps (fixed warp order) of per-lane-row values va_, vb_
+    auto exchange = [&](float &pa_, float &pb_, int v, bool is_max) {
+      if (tq == 0) {
+        xs[(ns * 16 + g) * 2 + v] = pa_;
+        xs[(ns * 16 + g + 8) * 2 + v] = pb_;
+      }
+      tile_bar();
+      float ta = xs[(0 * 16 + g) * 2 + v], tb = xs[(0 * 16 + g + 8) * 2 + v];
+#pragma unroll
+      for (int q = 1; q < WPT; ++q) {
+        const float xa_ = xs[(q * 16 + g) * 2 + v], xb_ = xs[(q * 16 + g + 8) * 2 + v];
+        ta = is_max ? fmaxf(ta, xa_) : ta + xa_;
+        tb = is_max ? fmaxf(tb, xb_) : tb + xb_;
+      }
+      pa_ = ta;
+      pb_ = tb;
+    };
     if (EPI == G_NODE) {
       // a2: h̄ = LReLU(.), p = h̄·a_s, q = h̄·a_d
       float pa = 0.f, qa = 0.f, pb = 0.f, qb = 0.f;
 #pragma unroll
-      for (int nt = 0; nt < NT; ++nt)
+      for (int nt = 0; nt < NTW; ++nt)
 #pragma unroll
         for (int h = 0; h < 2; ++h) {
-          const int col = nt * 8 + 2 * tq + h;
+          const int col = (ns * NTW + nt) * 8 + 2 * tq + h;
           const float oa = lrelu_s(c[nt][h], ep.slope), ob = lrelu_s(c[nt][2 + h], ep.slope);
           c[nt][h] = oa;
           c[nt][2 + h] = ob;
@@ -176,16 +210,19 @@ __device__ __forceinline__ void tgemm(const float *X, int ldx, const int32_t *xm
         pb += __shfl_xor_sync(0xffffffffu, pb, o);
         qb += __shfl_xor_sync(0xffffffffu, qb, o);
       }
-      if (tq == 0) {
+      exchange(pa, pb, 0, false);
+      exchange(qa, qb, 1, false);          // v = 1: same barrier phase sequence in every warp
+      if (ns == 0 && tq == 0) {
         if (va) { ep.pq[ra] = pa; ep.pq[SNMAX + ra] = qa; }
         if (vb) { ep.pq[rb] = pb; ep.pq[SNMAX + rb] = qb; }
       }
+      tile_bar();                          // xs is reused by the next m-tile on this slot
     } else if (EPI == G_EDGE) {
       // a3: e' = σ(α z), α = p[src] + q[dst]
       const float ala = ep.pq[ep.isrc[ia]] + ep.pq[SNMAX + ep.idst[ia]];
       const float alb = ep.pq[ep.isrc[ib]] + ep.pq[SNMAX + ep.idst[ib]];
 #pragma unroll
-      for (int nt = 0; nt < NT; ++nt)
+      for (int nt = 0; nt < NTW; ++nt)
 #pragma unroll
         for (int h = 0; h < 2; ++h) {
           c[nt][h] = __fdividef(1.f, 1.f + ex2_fast(-ala * c[nt][h] * LOG2E_S));
@@ -195,7 +232,7 @@ __device__ __forceinline__ void tgemm(const float *X, int ldx, const int32_t *xm
       // a4: g = softmax over the D channels of the logits (rows g and g+8)
       float ma = -INFINITY, mb = -INFINITY;
 #pragma unroll
-      for (int nt = 0; nt < NT; ++nt) {
+      for (int nt = 0; nt < NTW; ++nt) {
         ma = fmaxf(ma, fmaxf(c[nt][0], c[nt][1]));
         mb = fmaxf(mb, fmaxf(c[nt][2], c[nt][3]));
       }
@@ -204,9 +241,10 @@ __device__ __forceinline__ void tgemm(const float *X, int ldx, const int32_t *xm
         ma = fmaxf(ma, __shfl_xor_sync(0xffffffffu, ma, o));
         mb = fmaxf(mb, __shfl_xor_sync(0xffffffffu, mb, o));
       }
+      exchange(ma, mb, 0, true);
       float sa = 0.f, sb = 0.f;
 #pragma unroll
-      for (int nt = 0; nt < NT; ++nt)
+      for (int nt = 0; nt < NTW; ++nt)
 #pragma unroll
         for (int h = 0; h < 2; ++h) {
           c[nt][h] = ex2_fast((c[nt][h] - ma) * LOG2E_S);
@@ -219,9 +257,11 @@ __device__ __forceinline__ void tgemm(const float *X, int ldx, const int32_t *xm
         sa += __shfl_xor_sync(0xffffffffu, sa, o);
         sb += __shfl_xor_sync(0xffffffffu, sb, o);
       }
+      exchange(sa, sb, 1, false);
+      tile_bar();                          // xs is reused by the next m-tile on this slot
       const float inva = 1.f / sa, invb = 1.f / sb;
 #pragma unroll
-      for (int nt = 0; nt < NT; ++nt)
+      for (int nt = 0; nt < NTW; ++nt)
 #pragma unroll
         for (int h = 0; h < 2; ++h) {
           c[nt][h] *= inva;
@@ -229,8 +269,8 @@ __device__ __forceinline__ void tgemm(const float *X, int ldx, const int32_t *xm
         }
     }
 #pragma unroll
-    for (int nt = 0; nt < NT; ++nt) {
-      const int col = nt * 8 + 2 * tq;
+    for (int nt = 0; nt < NTW; ++nt) {
+      const int col = (ns * NTW + nt) * 8 + 2 * tq;
       if (va) *reinterpret_cast<float2 *>(Y + ra * ldy + col) = make_float2(c[nt][0], c[nt][1]);
       if (vb) *reinterpret_cast<float2 *>(Y + rb * ldy + col) = make_float2(c[nt][2], c[nt][3]);
     }
@@ -255,7 +295,9 @@ __global__ void __launch_bounds__(ST, 1) small_forward_kernel(const SmallArgs a)
   float *Rs = W1s + dh * (D + 4) + 2 * dh + 4; // [B][D] readout
   float *Cs = Rs + B * D;                      // [B][d_h] head hidden
   float *Av = Cs + B * dh;                     // [L][2][D] attention vectors a_s, a_d
-  int32_t *cs = reinterpret_cast<int32_t *>(Av + a.L * 2 * D);
+  float *Xr = Av + a.L * 2 * D;                // GEMM row-partial exchange (XR_FLOATS)
+  float *Rp = Xr + XR_FLOATS;                  // readout partials [P][B][D], P·B·D <= 4·ST
+  int32_t *cs = reinterpret_cast<int32_t *>(Rp + 4 * ST);
   int32_t *iptr = cs, *isrc = cs + (N + 1), *idst = isrc + E, *ieid = idst + E, *noff = ieid + E;
   const int t = threadIdx.x, warp = t >> 5, lane = t & 31;
 #ifdef OCCU_SMALL_TIMING
@@ -299,7 +341,7 @@ __global__ void __launch_bounds__(ST, 1) small_forward_kernel(const SmallArgs a)
   const float *Ein = Ef;
   int lde = a.F_e;
   float *Eout = Ea;
-  GemmEpi ep{a.slope, nullptr, pq, isrc, idst};
+  GemmEpi ep{a.slope, nullptr, pq, isrc, idst, Xr};
   for (int l = 0; l < a.L; ++l) {
     const float *P = a.P;
     // a2 (groups pending: layer 0 — group 0, W_u, W_e; later — W_e(l), W_u(l))
@@ -347,29 +389,34 @@ __global__ void __launch_bounds__(ST, 1) small_forward_kernel(const SmallArgs a)
     Eout = Eout == Ea ? Eb : Ea;
     K = D;
   }
-  // a7: per-graph mean readout (ascending nodes); a8: head, thread per hidden unit (W_1 rows
-  // padded to D + 1: conflict-free), then warp per graph for the final dot
-  for (int i = t; i < B * (D / 4); i += ST) {
-    const int b = i / (D / 4), c = 4 * (i % (D / 4));
-    const int u0 = noff[b], u1 = noff[b + 1];
-    float4 s[4];
-#pragma unroll
-    for (int q = 0; q < 4; ++q) s[q] = make_float4(0.f, 0.f, 0.f, 0.f);
-    for (int u = u0; u < u1; u += 4)
-#pragma unroll
-      for (int q = 0; q < 4; ++q)
-        if (u + q < u1) {
-          const float4 h = *reinterpret_cast<const float4 *>(H + (u + q) * SK + c);
-          s[q].x += h.x; s[q].y += h.y; s[q].z += h.z; s[q].w += h.w;
-        }
-    const float n = float(u1 - u0);
-    float4 o;
-    o.x = ((s[0].x + s[1].x) + (s[2].x + s[3].x)) / n;
-    o.y = ((s[0].y + s[1].y) + (s[2].y + s[3].y)) / n;
-    o.z = ((s[0].z + s[1].z) + (s[2].z + s[3].z)) / n;
-    o.w = ((s[0].w + s[1].w) + (s[2].w + s[3].w)) / n;
-    *reinterpret_cast<float4 *>(Rs + b * D + c) = o;
-    *reinterpret_cast<float4 *>(a.r + b * D + c) = o;
+  // a7: per-graph mean readout in two levels: P node-strided partial sums per (graph, 4
+  // channels) over all threads, then the P partials in fixed order (one serial chain of
+  // ~N/P instead of N shared-memory round trips); a8: head, thread per hidden unit (W_1 rows
+  // padded to D + 4), then warp per graph for the final dot
+  {
+    const int BC = B * (D / 4), P = max(1, min(32, ST / BC));
+    for (int i = t; i < P * BC; i += ST) {
+      const int p = i / BC, j = i - p * BC, b = j / (D / 4), c = 4 * (j % (D / 4));
+      float4 s = make_float4(0.f, 0.f, 0.f, 0.f);
+      for (int u = noff[b] + p; u < noff[b + 1]; u += P) {
+        const float4 h = *reinterpret_cast<const float4 *>(H + u * SK + c);
+        s.x += h.x; s.y += h.y; s.z += h.z; s.w += h.w;
+      }
+      *reinterpret_cast<float4 *>(Rp + (p * B + b) * D + c) = s;
+    }
+    __syncthreads();
+    for (int i = t; i < BC; i += ST) {
+      const int b = i / (D / 4), c = 4 * (i % (D / 4));
+      float4 s = make_float4(0.f, 0.f, 0.f, 0.f);
+      for (int p = 0; p < P; ++p) {
+        const float4 h = *reinterpret_cast<const float4 *>(Rp + (p * B + b) * D + c);
+        s.x += h.x; s.y += h.y; s.z += h.z; s.w += h.w;
+      }
+      const float n = float(noff[b + 1] - noff[b]);
+      const float4 o = make_float4(s.x / n, s.y / n, s.z / n, s.w / n);
+      *reinterpret_cast<float4 *>(Rs + b * D + c) = o;
+      *reinterpret_cast<float4 *>(a.r + b * D + c) = o;
+    }
   }
   __syncthreads(); STAMP(8);
   for (int o = t; o < B * dh; o += ST) {
@@ -416,7 +463,7 @@ static size_t small_smem(const occu_config &c, const DevCsr &csr) {
   const int sk = small_sk(c), ld = c.d + 4;
   return size_t(csr.N * sk + csr.N * ld + 2 * SNMAX + csr.E * c.F_e + 3 * csr.E * ld +
                 2 * c.d * (small_kw(c) + 4) + c.d_h * (c.d + 4) + 2 * c.d_h + 4 + csr.B * (c.d + c.d_h) +
-                c.L * 2 * c.d + (csr.N + 1) + 3 * csr.E + (csr.B + 1)) * 4;
+                c.L * 2 * c.d + XR_FLOATS + 4 * ST + (csr.N + 1) + 3 * csr.E + (csr.B + 1)) * 4;
 }
 
 bool small_forward_ok(const occu_ctx *ctx, const DevCsr &csr) {

@@ -1,0 +1,40 @@
+"""The training step's byte-saving variants against the paths they replace (same process
+code, A/B by the library's environment switches, each run in its own subprocess):
+
+* LReLU'(h) from the forward's sign bits (default) vs from the stored h rows
+  (OCCU_NO_HBITS=1): the same per-element decisions, so the gradient is BITWISE equal;
+* dα by the compensated FP32 dot (default) vs float64 FMAs (OCCU_DA_F64=1): both are
+  accurate far beyond FP32 rounding of the result, so the gradients agree to ~1e-6.
+"""
+import os
+import subprocess
+import sys
+
+import numpy as np
+import pytest
+
+pytestmark = pytest.mark.gpu
+HERE = os.path.dirname(os.path.abspath(__file__))
+
+
+def grads(tmp_path, tag, **env):
+    out = str(tmp_path / f"{tag}.npy")
+    e = dict(os.environ)
+    e.update(env)
+    subprocess.run([sys.executable, os.path.join(HERE, "_ab_grads.py"), out], env=e, check=True,
+                   timeout=600)
+    return np.load(out)
+
+
+@pytest.mark.parametrize("prec,aggr", [("f32", 0), ("f32", 1), ("bf16", 0)])
+def test_sign_bits_mask_is_bitwise_the_row_mask(tmp_path, prec, aggr):
+    a = grads(tmp_path, "bits", AB_PREC=prec, AB_AGGR=str(aggr))
+    b = grads(tmp_path, "rows", AB_PREC=prec, AB_AGGR=str(aggr), OCCU_NO_HBITS="1")
+    assert np.array_equal(a, b)
+
+
+def test_dot2_dalpha_matches_float64(tmp_path):
+    a = grads(tmp_path, "dot2")
+    b = grads(tmp_path, "f64", OCCU_DA_F64="1")
+    rel = np.abs(a - b) / np.maximum(np.abs(b), 1e-3 * np.abs(b).max())
+    assert rel.max() < 1e-5, rel.max()
