@@ -84,15 +84,15 @@ __device__ __forceinline__ void cpa_wait() { asm volatile("cp.async.wait_group %
 __device__ __noinline__ void stage_rows(float *dst, int sld, const float *__restrict__ src, int gld,
                                         int rows, int cols) {
   if ((reinterpret_cast<uintptr_t>(src) & 15) == 0 && gld % 4 == 0 && sld % 4 == 0) {
-    const uint32_t c4 = uint32_t(cols) / 4, magic = 0xFFFFFFFFu / c4 + 1u;
+    const uint32_t c4 = uint32_t(cols) / 4, magic = 0xFFFFFFFFu / c4 + 1u;   // c4 = 1: magic wraps to 0
     for (uint32_t i = threadIdx.x; i < uint32_t(rows) * c4; i += ST) {
-      const uint32_t n = __umulhi(i, magic), k = 4u * (i - n * c4);
+      const uint32_t n = c4 == 1u ? i : __umulhi(i, magic), k = 4u * (i - n * c4);
       cpa16(dst + n * sld + k, src + long(n) * gld + k);
     }
   } else {
     const uint32_t magic = 0xFFFFFFFFu / uint32_t(cols) + 1u;
     for (uint32_t i = threadIdx.x; i < uint32_t(rows) * uint32_t(cols); i += ST) {
-      const uint32_t n = __umulhi(i, magic), k = i - n * uint32_t(cols);
+      const uint32_t n = cols == 1 ? i : __umulhi(i, magic), k = i - n * uint32_t(cols);
       cpa4(dst + n * sld + k, src + long(n) * gld + k);
     }
   }

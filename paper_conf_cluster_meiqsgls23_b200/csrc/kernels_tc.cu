@@ -1432,9 +1432,17 @@ struct EdgeGateArgs {
   const int *wf_e, *wf_m;            // scale exponents (wf_m[1] = softmax no-shift flag)
   const float *p, *q;
   const int32_t *src, *dst;
-  float *e_out, *e0_out, *g;
+  float *e_out, *e0_out, *g;        // e_out nullable (last inference layer: e' is not needed)
   int rev;
   int dbg;                           // sensitivity experiments only (OCCU_EG_DBG), 0 in production
+  // AGG (a4 + a5 + a6 fused into stage 2, inference): m = g ⊙ h̄[s] summed over each
+  // destination's dst-sorted in-edges inside the warp's 32 rows; complete segments -> h_out
+  // (LReLU, ÷ deg for MEAN), segments crossing a 32-edge unit -> part (agg_fixup_kernel)
+  const float *hbar;
+  const int32_t *in_ptr;
+  float *h_out, *part;
+  int mean;
+  float slope;
 };
 
 constexpr int EG_NTH = 832;
@@ -1446,7 +1454,7 @@ __host__ __device__ inline size_t eg_smem_bytes(int D, int Ke, bool first) {
   return 1024 + 2 * imgm + 2 * imge + ring + 256 + 2 * 2 * 128 * 4 + 16 * 16 * 20 * 4;
 }
 
-template <int D, int KM>      // KM > 0: FIRST (layer-1 CUDA-core edge transform, Ke <= KM)
+template <int D, int KM, bool AGG = false>   // KM > 0: FIRST (layer-1 CUDA-core edge transform, Ke <= KM)
 __global__ void __launch_bounds__(EG_NTH, 1) edgegate_kernel(const __grid_constant__ CUtensorMap tmap,
                                                              EdgeGateArgs a) {
   constexpr bool FIRST = KM > 0;
@@ -1716,7 +1724,7 @@ __global__ void __launch_bounds__(EG_NTH, 1) edgegate_kernel(const __grid_consta
         const uint32_t col = A2 + uint32_t((cb + c0) / 2);
         tc::tmem_st8(lane_base + col, x0);
         tc::tmem_st8(lane_base + col + D / 2, x1);
-        if (!(a.dbg & 4)) warp_store_chunk<D>(wbuf, a.e_out, wrow0, wrows, cb + c0, o, lane);
+        if (!(a.dbg & 4) && a.e_out) warp_store_chunk<D>(wbuf, a.e_out, wrow0, wrows, cb + c0, o, lane);
       }
       tc::tmem_st_wait();
       tc::fence_before_sync();
@@ -1773,6 +1781,80 @@ __global__ void __launch_bounds__(EG_NTH, 1) edgegate_kernel(const __grid_consta
       group_bar(1);
       sum = hf == 0 ? sum + xg[256 + 128 + row] : xg[256 + row] + sum;   // fixed order
       const float inv = fast_rcp(sum);
+      if constexpr (AGG) {
+        // destination segments inside this warp's 32 consecutive (dst-sorted) edges
+        const long grow = r0 + row;
+        const bool live = row < nrows;
+        const int tn = live ? __ldg(a.dst + grow) : -1 - lane;         // pad rows: own segment
+        const int sn = live ? __ldg(a.src + grow) : 0;
+        const int tprev = __shfl_up_sync(0xffffffffu, tn, 1);
+        const int tnext = __shfl_down_sync(0xffffffffu, tn, 1);
+        const bool head = lane == 0 || tprev != tn;
+        const bool tail = lane == 31 || tnext != tn;
+        const unsigned heads = __ballot_sync(0xffffffffu, head);
+        const int start = 31 - __clz(heads & (0xffffffffu >> (31 - lane)));
+        const int maxlen = __reduce_max_sync(0xffffffffu, unsigned(lane - start + 1));
+        int beg = 0, end = 0;
+        if (tail && live) {
+          beg = __ldg(a.in_ptr + tn);
+          end = __ldg(a.in_ptr + tn + 1);
+        }
+        const bool before = live && beg < wrow0 + start;               // segment began earlier
+        const bool after = live && end > wrow0 + lane + 1;               // continues after this warp
+        const float dsc = a.mean ? float(end - beg > 0 ? end - beg : 1) : 1.f;
+        const float *hbr = a.hbar + long(sn) * D + cb;
+        const long unit = wrow0 >> 5;
+        float4 hpre[4];                                                  // h̄[s] one chunk ahead
+#pragma unroll
+        for (int u = 0; u < 4; ++u)
+          hpre[u] = live ? __ldg(reinterpret_cast<const float4 *>(hbr) + u) : make_float4(0.f, 0.f, 0.f, 0.f);
+#pragma unroll 1
+        for (int c0 = 0; c0 < DH; c0 += 16) {
+          uint32_t r[16];
+          tc::tmem_ld16(acc + c0, r);
+          float4 hc[4];
+#pragma unroll
+          for (int u = 0; u < 4; ++u) hc[u] = hpre[u];
+          if (c0 + 16 < DH)
+#pragma unroll
+            for (int u = 0; u < 4; ++u)
+              hpre[u] = live ? __ldg(reinterpret_cast<const float4 *>(hbr + c0 + 16) + u) : make_float4(0.f, 0.f, 0.f, 0.f);
+          tc::tmem_ld_wait();
+          float v[16];
+#pragma unroll
+          for (int u = 0; u < 16; u += 4) {
+            const float bv[4] = {hc[u >> 2].x, hc[u >> 2].y, hc[u >> 2].z, hc[u >> 2].w};
+#pragma unroll
+            for (int t = 0; t < 4; ++t)                                 // m = g ⊙ h̄[s]
+              v[u + t] = ex2(fmaf(__uint_as_float(r[u + t]), unL, -mL)) * inv * bv[t];
+          }
+          // segmented inclusive scan across lanes (fixed tree order)
+          for (int d = 1; d < maxlen; d <<= 1) {        // only as many steps as the longest run
+#pragma unroll
+            for (int u = 0; u < 16; ++u) {
+              const float o = __shfl_up_sync(0xffffffffu, v[u], d);
+              if (lane - d >= start) v[u] += o;
+            }
+          }
+          if (tail && live) {
+            if (!before && !after) {                                   // complete segment
+              float *hr = a.h_out + long(tn) * D + cb + c0;
+#pragma unroll
+              for (int u = 0; u < 16; u += 4) {
+                float o4[4];
+#pragma unroll
+                for (int t = 0; t < 4; ++t) o4[t] = lrelu(a.mean ? v[u + t] / dsc : v[u + t], a.slope);
+                *reinterpret_cast<float4 *>(hr + u) = make_float4(o4[0], o4[1], o4[2], o4[3]);
+              }
+            } else {
+              float *pr = a.part + (unit * 2 + (before ? 0 : 1)) * D + cb + c0;
+#pragma unroll
+              for (int u = 0; u < 16; u += 4)
+                *reinterpret_cast<float4 *>(pr + u) = make_float4(v[u], v[u + 1], v[u + 2], v[u + 3]);
+            }
+          }
+        }
+      } else
 #pragma unroll 1
       for (int c0 = 0; c0 < DH; c0 += 16) {
         uint32_t r[16];
@@ -2502,10 +2584,13 @@ static int tc_forward_layer_pair(const occu_ctx *ctx, const DevCsr &csr, int lay
 
 template <int D>
 static int launch_edgegate(const occu_ctx *ctx, const DevCsr &csr, int layer, const FwdLayerArgs &a,
-                           cudaStream_t st) {
+                           cudaStream_t st, float *partial = nullptr) {
   if (csr.E <= 0) return 0;
   const bool first = a.Ke <= 16;
+  const bool agg = partial != nullptr;
   EdgeGateArgs ea{};
+  ea.hbar = a.hbar; ea.in_ptr = csr.in_ptr; ea.h_out = a.h_out; ea.part = partial;
+  ea.mean = ctx->cfg.aggr == OCCU_AGGR_MEAN; ea.slope = ctx->cfg.slope;
   ea.e_in = a.e_in; ea.Ke = a.Ke; ea.R = csr.E; ea.eid = a.e_eid; ea.W_e = a.W_e;
   ea.wimg_m = tc_wimg(ctx, 2, layer); ea.wf_m = tc_wfexp(ctx, 2, layer);
   if (!first) {
@@ -2526,17 +2611,20 @@ static int launch_edgegate(const occu_ctx *ctx, const DevCsr &csr, int layer, co
   CUtensorMap tmap;
   memset(&tmap, 0, sizeof(tmap));
   if (!first && !encode_rows_map(&tmap, a.e_in, csr.E, a.Ke)) return -int(cudaErrorInvalidValue);
-  OCCU_PROF_BEGIN(ctx, "edge_gate_tc", st);
+  OCCU_PROF_BEGIN(ctx, agg ? "edge_gate_agg_tc" : "edge_gate_tc", st);
+#define OCCU_EG_LAUNCH(KMV, AGGV)                                                   \
+  do {                                                                            \
+    set_smem(edgegate_kernel<D, KMV, AGGV>, smem);                                \
+    edgegate_kernel<D, KMV, AGGV><<<grid, EG_NTH, smem, st>>>(tmap, ea);           \
+  } while (0)
   if (!first) {
-    set_smem(edgegate_kernel<D, 0>, smem);
-    edgegate_kernel<D, 0><<<grid, EG_NTH, smem, st>>>(tmap, ea);
+    if (agg) OCCU_EG_LAUNCH(0, true); else OCCU_EG_LAUNCH(0, false);
   } else if (a.Ke <= 4) {
-    set_smem(edgegate_kernel<D, 4>, smem);
-    edgegate_kernel<D, 4><<<grid, EG_NTH, smem, st>>>(tmap, ea);
+    if (agg) OCCU_EG_LAUNCH(4, true); else OCCU_EG_LAUNCH(4, false);
   } else {
-    set_smem(edgegate_kernel<D, 16>, smem);
-    edgegate_kernel<D, 16><<<grid, EG_NTH, smem, st>>>(tmap, ea);
+    if (agg) OCCU_EG_LAUNCH(16, true); else OCCU_EG_LAUNCH(16, false);
   }
+#undef OCCU_EG_LAUNCH
   OCCU_PROF_END(ctx);
   TC_CHECK();
   return 1;
@@ -2558,8 +2646,27 @@ static int tc_forward_layer_impl(const occu_ctx *ctx, const DevCsr &csr, int lay
   ra.rev = ctx->l2_order;
   if ((r = launch_rowgemm<D, EPI_NODE>(ctx, ra, "node_tc", st)) < 0) return r;
   n += r;
-  const bool fused_eg = ctx->path == 0 && ctx->fuse_edge_gate && ctx->cfg.msg == OCCU_MSG_CHANNEL_SOFTMAX &&
+  const bool eg_shape = ctx->path == 0 && ctx->cfg.msg == OCCU_MSG_CHANNEL_SOFTMAX &&
                         (a.Ke <= 16 || (a.Ke % 64 == 0 && a.Ke <= 128));
+  const bool fused_ega = eg_shape && a.infer;          // a3 + a4 + a5 + a6 (inference)
+  const bool fused_eg = eg_shape && ctx->fuse_edge_gate && !fused_ega;
+  if (fused_ega) {
+    // e' (unless last), then g ⊙ h̄[s] summed per destination inside each 32-edge unit: g never
+    // reaches HBM; segments crossing a unit boundary and nodes without in-edges are completed
+    // by agg_fixup_kernel from the unit partials (fixed unit order)
+    if (csr.E > 0 && (r = launch_edgegate<D>(ctx, csr, layer, a, st, partial)) < 0) return r;
+    n += csr.E > 0 ? r : 0;
+    if (csr.N > 0) {
+      const int grid = int(std::min<long>((long(csr.N) + 255) / 256, 8L * ctx->num_sms));
+      OCCU_PROF_BEGIN(ctx, "agg_fixup", st);
+      agg_fixup_kernel<<<grid, 256, 0, st>>>(csr.in_ptr, csr.N, D, partial,
+                                             ctx->cfg.aggr == OCCU_AGGR_MEAN, slope, a.h_out);
+      OCCU_PROF_END(ctx);
+      TC_CHECK();
+      ++n;
+    }
+    return n;
+  }
   if (csr.E > 0 && fused_eg) {
     // a3 + a4 fused: e' and g in one kernel (e' is not re-read)
     if ((r = launch_edgegate<D>(ctx, csr, layer, a, st)) < 0) return r;

@@ -126,6 +126,8 @@ struct occu_ctx {
   // gather.  Default from A/B runs on CFG2: the FP32 gather and the readout lose with it.
   int pdl = 1 | 4 | 16 | 32 | 64;
   int fuse_edge_gate = 0;  // path 0: edge transform + gate in one kernel (edgegate_kernel), OCCU_FUSE_EG=1
+  int fuse_agg = 0;        // path 0 inference: edge transform + gate + message + segmented sum in one
+                           // kernel (edgegate_kernel<AGG>; g never reaches HBM), OCCU_FUSE_EGA
   occu::DevBuf wimg, wjobs, wfexp;   // prebuilt tensor-core weight images (per parameter version)
   int64_t params_version = 0, wimg_version = -1;
   int64_t dprep_version = -1;   // decoder: params version the folded key map was built for
@@ -200,6 +202,7 @@ struct FwdLayerArgs {
   const int32_t *e_eid; float *e0_out; float *rpart;
   bool save_w = false;                 // reading B, training: g receives the softmax weights
   uint32_t *h_bits = nullptr;          // training: sign bitmask of h_out for the backward's LReLU'
+  bool infer = false;                  // inference (nothing saved): the fused edge-gate-aggregate kernel may run
 };
 int launch_forward_layer(const occu_ctx *ctx, const DevCsr &csr, const FwdLayerArgs &a,
                          cudaStream_t st);

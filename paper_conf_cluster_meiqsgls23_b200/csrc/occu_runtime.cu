@@ -282,7 +282,11 @@ occu_status forward(occu_ctx *ctx, const DevCsr &csr, const float *nf, const flo
   const bool fuse_e0 = tc && c.F_e <= 16;
   const bool dec = c.readout == OCCU_READOUT_SET_DECODER;
   const bool gph = c.graphormer > 0;
-  const bool fuse_ro = tc && (bf || ctx->path == 0) && !dec && !gph;
+  // inference on the fused edge-gate-aggregate kernel: h rows are written by that kernel and
+  // its boundary fixup (no readout chunk partials), the last layer's e' is not written at all
+  const bool ega = !save_all && !bf && tc && ctx->path == 0 && ctx->fuse_agg &&
+                   c.msg == OCCU_MSG_CHANNEL_SOFTMAX && (c.d == 64 || c.d == 128);
+  const bool fuse_ro = tc && (bf || ctx->path == 0) && !dec && !gph && !ega;
   if (!fuse_e0) LK(launch_permute_rows(ctx, ef, csr.in_eid, csr.E, c.F_e, w.e0.as<float>(), s), "permute e0");
   if (tc) LK(tc_prepare_weights(ctx, s), "weight images");
   float *rpart = nullptr;
@@ -323,8 +327,9 @@ occu_status forward(occu_ctx *ctx, const DevCsr &csr, const float *nf, const flo
       a.h_bits = reinterpret_cast<uint32_t *>(w.hbits[i].ptr);
       ctx->hbits_layers = i + 1;
     }
+    a.infer = ega;
     if (tc) {
-      a.e_out = w.e[i].as<float>();            // the gate kernel re-reads e'
+      a.e_out = (ega && last) ? nullptr : w.e[i].as<float>();   // the gate kernel re-reads e'
       if (last && fuse_ro) {
         a.rpart = rpart;
         if (!save_all) a.h_out = nullptr;
@@ -635,6 +640,7 @@ occu_status occu_create(occu_ctx **out, const occu_config *cfg, int cuda_device,
   cudaDeviceGetAttribute(&ctx->num_sms, cudaDevAttrMultiProcessorCount, cuda_device);
   if (const char *e = getenv("OCCU_L2_ORDER")) ctx->l2_order = atoi(e);   // A/B switches
   if (const char *e = getenv("OCCU_FUSE_EG")) ctx->fuse_edge_gate = atoi(e);
+  if (const char *e = getenv("OCCU_FUSE_EGA")) ctx->fuse_agg = atoi(e);
   if (const char *e = getenv("OCCU_PDL")) ctx->pdl = atoi(e);
   const size_t pb = (ctx->layout.total + 1) * 4;
   if (ctx->params.ensure(pb) != cudaSuccess || ctx->grads.ensure(pb) != cudaSuccess ||

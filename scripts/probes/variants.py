@@ -62,10 +62,12 @@ def infer():
     nf = torch.from_numpy(b.node_feat).to(dev)
     ef = torch.from_numpy(b.edge_feat).to(dev)
     for prec, pname in ((occu.FP32, "f32"), (occu.BF16, "bf16")):
-        for tag, path, env in (("path0", 0, {}), ("path2", 2, {}), ("fuse_eg", 0, {"OCCU_FUSE_EG": "1"})):
+        for tag, path, env in (("path0", 0, {}), ("path2", 2, {}), ("fuse_eg", 0, {"OCCU_FUSE_EG": "1"}),
+                               ("fuse_ega", 0, {"OCCU_FUSE_EGA": "1"}), ("path0_again", 0, {})):
             if prec == occu.BF16 and path == 2:
                 continue
             os.environ.pop("OCCU_FUSE_EG", None)
+            os.environ.pop("OCCU_FUSE_EGA", None)
             os.environ.update(env)
             m = occu.Model(occu.config(L=3, F_n=80, F_e=4, d=128, prec=prec))
             m.init_weights(42)
@@ -76,6 +78,7 @@ def infer():
             show(f"CFG2 infer {pname} {tag}", ms, prof)
             del m
     os.environ.pop("OCCU_FUSE_EG", None)
+    os.environ.pop("OCCU_FUSE_EGA", None)
 
 
 def train():
