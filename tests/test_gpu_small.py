@@ -53,3 +53,25 @@ def test_small_forward_matches_oracle_and_regular_path(L, d, aggr, ng, seed):
     assert np.allclose(y_small, y_reg, rtol=1e-5, atol=1e-7)
     m.keep_intermediates(False)
     assert np.array_equal(m.predict(csr, b.node_feat, b.edge_feat), y_small)    # deterministic
+
+
+def test_small_forward_repeatable_under_repetition():
+    """Race probe for the single-CTA kernel (named-barrier row exchange between the 4 warps of
+    an m-tile, cp.async staging groups, two-level readout): 300 launches on the same inputs
+    must give bitwise the same outputs (compute-sanitizer is not available on this pool)."""
+    import torch
+    c = occu.config(L=2, F_n=80, F_e=4, d=64)
+    b = configs.cfg1()
+    m = occu.Model(c)
+    m.init_weights(7)
+    m.set_small_batch_kernel(True)
+    dev = torch.device("cuda", 0)
+    csr = m.to_device(occu.pack(b.graphs))
+    nf = torch.from_numpy(b.node_feat).to(dev)
+    ef = torch.from_numpy(b.edge_feat).to(dev)
+    outs = torch.empty(300, dtype=torch.float32, device=dev)
+    for i in range(300):
+        m.predict(csr, nf, ef, outs[i:i + 1])
+    assert m.last_launch_count() == 1
+    o = outs.cpu().numpy()
+    assert np.all(o == o[0]), np.unique(o)
