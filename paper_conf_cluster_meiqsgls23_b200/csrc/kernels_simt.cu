@@ -609,8 +609,10 @@ __global__ void __launch_bounds__(NT) hub_merge_kernel(const int32_t *__restrict
   }
 }
 
-template <int D, int G, bool RP, bool BF = false, bool PF = false>
-__global__ void __launch_bounds__(NT, (BF ? G <= 8 : (G == 4 && !RP)) ? 4 : 3) gather_segsum_v2_kernel(
+// HB: training forward — also write the sign bits of h (hbits); a separate instantiation so that
+// the inference kernels carry none of its registers
+template <int D, int G, bool RP, bool BF = false, bool PF = false, bool HB = false>
+__global__ void __launch_bounds__(NT, (BF ? G <= 8 : (G == 4 && !RP && !HB)) ? 4 : 3) gather_segsum_v2_kernel(
     const void *__restrict__ g, const void *__restrict__ hbar,
     const int32_t *__restrict__ in_ptr, const int32_t *__restrict__ in_src, int N, int mean,
     float slope, void *__restrict__ h_out, const int32_t *__restrict__ node_graph,
@@ -659,7 +661,7 @@ __global__ void __launch_bounds__(NT, (BF ? G <= 8 : (G == 4 && !RP)) ? 4 : 3) g
         acc[c] = 0.f;
       }
       if (!RP || h_out) store_row_t<V, BF>(h_out, t0 + nd, D, lane, o);
-      if (hbits) {      // word c, bit l: channel V·l + c is positive (LReLU' = 1)
+      if constexpr (HB) {      // word c, bit l: channel V·l + c is positive (LReLU' = 1)
         uint32_t mine = 0u;
 #pragma unroll
         for (int c = 0; c < V; ++c) {
@@ -2031,7 +2033,12 @@ static int gather_impl(const occu_ctx *ctx, const DevCsr &csr, const float *g, c
   OCCU_PROF_BEGIN(ctx, "gather_segsum", st);
 #define OCCU_GATHER_ARGS g, hbar, csr.in_ptr, csr.in_src, csr.N, mean, ctx->cfg.slope, h_out, csr.node_graph, rpart, hub, csr.in_dst, hbits
   if (hbits && variant != 1) return -int(cudaErrorInvalidValue);    // sign bits: default kernel only
-  if constexpr (D == 256) {
+  if (hbits) {                // training forward: the sign-bit variants
+    const int grid = grid_for(long(csr.N) * 4, NT, occ * ctx->num_sms);
+    constexpr int GG = D == 256 ? 2 : 4;
+    if (rpart) launch_pdl(ctx->pdl & 2, gather_segsum_v2_kernel<D, GG, true, false, false, true>, grid, NT, 0, st, OCCU_GATHER_ARGS);
+    else launch_pdl(ctx->pdl & 2, gather_segsum_v2_kernel<D, GG, false, false, false, true>, grid, NT, 0, st, OCCU_GATHER_ARGS);
+  } else if constexpr (D == 256) {
     // d = 256: two (g, h̄) row pairs in flight per lane (16 floats each); 1 KB rows
     const int grid = grid_for(long(csr.N) * 4, NT, occ * ctx->num_sms);
     if (rpart) launch_pdl(ctx->pdl & 2, gather_segsum_v2_kernel<D, 2, true>, grid, NT, 0, st, OCCU_GATHER_ARGS);
@@ -2083,7 +2090,11 @@ static int gather_bf16_impl(const occu_ctx *ctx, const DevCsr &csr, const void *
   if (r0 < 0) return r0;
   OCCU_PROF_BEGIN(ctx, "gather_segsum", st);
 #define OCCU_GB_ARGS g, hbar, csr.in_ptr, csr.in_src, csr.N, mean, ctx->cfg.slope, h_out, csr.node_graph, rpart, hub, csr.in_dst, hbits
-  if constexpr (D == 256) {
+  if (hbits) {                // training forward: the sign-bit variants
+    constexpr int GG = D == 256 ? 2 : 4;
+    if (rpart) launch_pdl(ctx->pdl & 64, gather_segsum_v2_kernel<D, GG, true, true, false, true>, grid, NT, 0, st, OCCU_GB_ARGS);
+    else launch_pdl(ctx->pdl & 64, gather_segsum_v2_kernel<D, GG, false, true, false, true>, grid, NT, 0, st, OCCU_GB_ARGS);
+  } else if constexpr (D == 256) {
     if (rpart) launch_pdl(ctx->pdl & 64, gather_segsum_v2_kernel<D, 2, true, true>, grid, NT, 0, st, OCCU_GB_ARGS);
     else launch_pdl(ctx->pdl & 64, gather_segsum_v2_kernel<D, 2, false, true>, grid, NT, 0, st, OCCU_GB_ARGS);
   } else if (gsel == 4) {
