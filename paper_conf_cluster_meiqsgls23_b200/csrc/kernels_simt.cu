@@ -2431,10 +2431,12 @@ static int backward_layer_impl(occu_ctx *ctx, const DevCsr &csr, const BwdLayerA
 #define OCCU_EBS_ARGS a.e_in, a.Ke, a.e, de, P + L.W_e[i], a.p, a.q, csr.in_src, csr.in_dst, csr.E, \
     w.DZ.as<float>(), w.dalpha.as<float>()
       if (a.Ke == 4 && fuse_we) {
-        // layer 1 with F_e = 4: dW_e accumulated here (per-block partials in the W_e slot)
-        if (bf) edge_bwd_small_kernel<D, 4, true, true><<<eg, NT, 0, st>>>(OCCU_EBS_ARGS, slot + WG_SLOT_FLOATS);
-        else edge_bwd_small_kernel<D, 4, false, true><<<eg, NT, 0, st>>>(OCCU_EBS_ARGS, slot + WG_SLOT_FLOATS);
-        we_blocks = eg;
+        // layer 1 with F_e = 4: dW_e accumulated here (per-block partials in the W_e slot); one
+        // wave of resident blocks (each reduces its partial once) instead of several
+        const int egw = grid_for((long(csr.E) + 31) / 32, NT / 32, 2 * sms);
+        if (bf) edge_bwd_small_kernel<D, 4, true, true><<<egw, NT, 0, st>>>(OCCU_EBS_ARGS, slot + WG_SLOT_FLOATS);
+        else edge_bwd_small_kernel<D, 4, false, true><<<egw, NT, 0, st>>>(OCCU_EBS_ARGS, slot + WG_SLOT_FLOATS);
+        we_blocks = egw;
       } else if (a.Ke <= 4) {
         if (bf) edge_bwd_small_kernel<D, 4, true><<<eg, NT, 0, st>>>(OCCU_EBS_ARGS);
         else edge_bwd_small_kernel<D, 4, false><<<eg, NT, 0, st>>>(OCCU_EBS_ARGS);
