@@ -804,7 +804,10 @@ __global__ void __launch_bounds__(NT) gate_bwd_stream_kernel(
     const void *__restrict__ g, const float *__restrict__ dA, const void *__restrict__ hbar,
     const int32_t *__restrict__ in_src, const int32_t *__restrict__ in_dst, int E,
     float *__restrict__ MG, float *__restrict__ DV, const float *__restrict__ h = nullptr,
-    const int32_t *__restrict__ in_ptr = nullptr, int mean = 0, float slope = 0.01f) {
+    const int32_t *__restrict__ in_ptr = nullptr, int mean = 0, float slope = 0.01f,
+    int *__restrict__ dv_rexp = nullptr) {
+  // dv_rexp: the fp16x2 scale exponent of each DV row (max |DV| over the row), read by the
+  // W_m row-GEMM's converters instead of a row-max pass of their own
   constexpr int V = D / 32;
   constexpr int G = 4;
   const int lane = threadIdx.x & 31;
@@ -870,6 +873,13 @@ __global__ void __launch_bounds__(NT) gate_bwd_stream_kernel(
         }
         if (MG) store_row<V>(MG + (k0 + j + u) * D + lane * V, mg);
         store_row<V>(DV + (k0 + j + u) * D + lane * V, dvv);
+        if (dv_rexp) {        // row max |DV|: one warp integer max-reduce of the |x| bit patterns
+          float mx = 0.f;
+#pragma unroll
+          for (int c = 0; c < V; ++c) mx = fmaxf(mx, fabsf(dvv[c]));
+          mx = __uint_as_float(__reduce_max_sync(0xffffffffu, __float_as_uint(mx)));
+          if (lane == 0) dv_rexp[k0 + j + u] = occu_row_scale_exp(mx);
+        }
       }
     }
   }
@@ -1642,7 +1652,8 @@ __global__ void __launch_bounds__(NT, FROMG ? 2 : 3) node_bwd_v2_kernel(
     const int32_t *__restrict__ out_ptr, const int32_t *__restrict__ out_pos,
     const int32_t *__restrict__ in_ptr, int N, float slope, float *__restrict__ dP,
     float *__restrict__ dpq, float *__restrict__ da_part, const void *__restrict__ gsv,
-    const float *__restrict__ dA, const int32_t *__restrict__ in_dst) {
+    const float *__restrict__ dA, const int32_t *__restrict__ in_dst, int *__restrict__ dp_rexp) {
+  // dp_rexp: the fp16x2 scale exponent of each dP row, for the dh_prev row-GEMM's converters
   constexpr int V = D / 32;
   constexpr int NPW = 8, G = 4;
   const int lane = threadIdx.x & 31;
@@ -1693,6 +1704,13 @@ __global__ void __launch_bounds__(NT, FROMG ? 2 : 3) node_bwd_v2_kernel(
       if (lane == 0) {
         dpq[2 * (t0 + nd)] = dp;
         dpq[2 * (t0 + nd) + 1] = dq;
+      }
+      if (dp_rexp) {          // row max |dP|: one warp integer max-reduce of the |x| bit patterns
+        float mx = 0.f;
+#pragma unroll
+        for (int c = 0; c < V; ++c) mx = fmaxf(mx, fabsf(o[c]));
+        mx = __uint_as_float(__reduce_max_sync(0xffffffffu, __float_as_uint(mx)));
+        if (lane == 0) dp_rexp[t0 + nd] = occu_row_scale_exp(mx);
       }
       dp = 0.f;
     };
@@ -2377,6 +2395,17 @@ static int backward_layer_impl(occu_ctx *ctx, const DevCsr &csr, const BwdLayerA
   float *slot = w.partial.as<float>();
   static const bool fuse_we = !getenv("OCCU_NO_FUSE_WE");   // A/B switch: dW_e in the layer-1 edge backward
   static const bool use_bits = !getenv("OCCU_NO_HBITS");     // A/B switch: LReLU'(h_in) from the sign bits
+  // row scale exponents of DV, DZ, dP handed from their producers to the row-GEMMs that read
+  // them (the same exponents the converters would compute: bitwise-neutral, A/B OCCU_NO_REXP)
+  static const bool use_rexp = !getenv("OCCU_NO_REXP");
+  int *dv_rexp = nullptr, *dz_rexp = nullptr, *dp_rexp = nullptr;
+  if (use_rexp && tc) {
+    if (w.rexp.ensure((2 * size_t(csr.E) + size_t(csr.N) + 4) * 4) != cudaSuccess) return -int(cudaErrorMemoryAllocation);
+    dv_rexp = w.rexp.as<int>();
+    dz_rexp = dv_rexp + csr.E;
+    dp_rexp = dz_rexp + csr.E;
+  }
+  int *dv_used = nullptr, *dz_used = nullptr;   // exponents actually written this layer
   int we_blocks = 0;                        // > 0: dW_e partials already written by edge_bwd_small
   // the streaming gate backward (saved gates) leaves MG = dA[t] ⊙ g to the node backward
   const bool mg_from_g = tc && a.g && !getenv("OCCU_NODE_BWD_V1");
@@ -2394,12 +2423,15 @@ static int backward_layer_impl(occu_ctx *ctx, const DevCsr &csr, const BwdLayerA
       ++n;
     } else if (a.g) {
       OCCU_PROF_BEGIN(ctx, "gate_bwd", st);
+      dv_used = dv_rexp;
       if (bf)
         gate_bwd_stream_kernel<D, true><<<grid_for((long(csr.E) + 31) / 32, NT / 32, 8 * sms), NT, 0, st>>>(
-            a.g, a.dh, a.hbar, csr.in_src, csr.in_dst, csr.E, MGo, w.DV.as<float>());
+            a.g, a.dh, a.hbar, csr.in_src, csr.in_dst, csr.E, MGo, w.DV.as<float>(), nullptr, nullptr, 0,
+            0.01f, dv_rexp);
       else
         gate_bwd_stream_kernel<D, false><<<grid_for((long(csr.E) + 31) / 32, NT / 32, 8 * sms), NT, 0, st>>>(
-            a.g, a.dh, a.hbar, csr.in_src, csr.in_dst, csr.E, MGo, w.DV.as<float>());
+            a.g, a.dh, a.hbar, csr.in_src, csr.in_dst, csr.E, MGo, w.DV.as<float>(), nullptr, nullptr, 0,
+            0.01f, dv_rexp);
       OCCU_PROF_END(ctx);
       LAUNCH_CHECK();
       ++n;
@@ -2409,7 +2441,7 @@ static int backward_layer_impl(occu_ctx *ctx, const DevCsr &csr, const BwdLayerA
       n += r;
     }
     if ((r = launch_plain_tc(ctx, w.DV.as<float>(), D, csr.E, 3, i, a.de_out, de,
-                             "de_tc", st)) < 0) return r;
+                             "de_tc", st, nullptr, nullptr, false, nullptr, dv_used)) < 0) return r;
     n += r;
     if (a.Ke > 16 && bf) {
       if ((r = launch_bwd_edge_bf16(ctx, csr, i, a.e_in, a.Ke, a.e, de, a.p, a.q,
@@ -2417,7 +2449,8 @@ static int backward_layer_impl(occu_ctx *ctx, const DevCsr &csr, const BwdLayerA
       n += r;
     } else if (a.Ke > 16) {
       if ((r = launch_bwd_edge_tc(ctx, csr, i, a.e_in, a.Ke, a.e, de, a.p, a.q,
-                                  w.DZ.as<float>(), w.dalpha.as<float>(), st)) < 0) return r;
+                                  w.DZ.as<float>(), w.dalpha.as<float>(), st, dz_rexp)) < 0) return r;
+      dz_used = dz_rexp;
       n += r;
     } else {
       const int tiles = (csr.E + BM - 1) / BM;
@@ -2451,7 +2484,7 @@ static int backward_layer_impl(occu_ctx *ctx, const DevCsr &csr, const BwdLayerA
     }
     if (a.de_prev) {
       if ((r = launch_plain_tc(ctx, w.DZ.as<float>(), D, csr.E, 4, i, nullptr,
-                               a.de_prev, "de_prev_tc", st)) < 0) return r;
+                               a.de_prev, "de_prev_tc", st, nullptr, nullptr, false, nullptr, dz_used)) < 0) return r;
       n += r;
     }
   } else if (csr.E > 0) {
@@ -2486,13 +2519,13 @@ static int backward_layer_impl(occu_ctx *ctx, const DevCsr &csr, const BwdLayerA
 #define OCCU_NB_ARGS w.MG.as<float>(), w.dalpha.as<float>(), a.hbar, P + L.a_s[i], P + L.a_d[i], csr.out_ptr, \
     csr.out_pos, csr.in_ptr, csr.N, cf.slope, w.dP.as<float>(), w.dpq.as<float>(), da_part
   if (fromg && bf)
-    node_bwd_v2_kernel<D, true, true><<<nb_blocks, NT, 0, st>>>(OCCU_NB_ARGS, a.g, a.dh, csr.in_dst);
+    node_bwd_v2_kernel<D, true, true><<<nb_blocks, NT, 0, st>>>(OCCU_NB_ARGS, a.g, a.dh, csr.in_dst, dp_rexp);
   else if (fromg)
-    node_bwd_v2_kernel<D, false, true><<<nb_blocks, NT, 0, st>>>(OCCU_NB_ARGS, a.g, a.dh, csr.in_dst);
+    node_bwd_v2_kernel<D, false, true><<<nb_blocks, NT, 0, st>>>(OCCU_NB_ARGS, a.g, a.dh, csr.in_dst, dp_rexp);
   else if (nbv && bf)
-    node_bwd_v2_kernel<D, true, false><<<nb_blocks, NT, 0, st>>>(OCCU_NB_ARGS, nullptr, nullptr, nullptr);
+    node_bwd_v2_kernel<D, true, false><<<nb_blocks, NT, 0, st>>>(OCCU_NB_ARGS, nullptr, nullptr, nullptr, dp_rexp);
   else if (nbv)
-    node_bwd_v2_kernel<D, false, false><<<nb_blocks, NT, 0, st>>>(OCCU_NB_ARGS, nullptr, nullptr, nullptr);
+    node_bwd_v2_kernel<D, false, false><<<nb_blocks, NT, 0, st>>>(OCCU_NB_ARGS, nullptr, nullptr, nullptr, dp_rexp);
   else if (bf)
     node_bwd_kernel<D, true><<<nb_blocks, NT, 0, st>>>(OCCU_NB_ARGS);
   else
@@ -2522,7 +2555,7 @@ static int backward_layer_impl(occu_ctx *ctx, const DevCsr &csr, const BwdLayerA
   if (a.dh_prev && csr.N > 0 && tc) {   // dh^{i-1} = dP W_u on tensor cores
     if ((r = launch_plain_tc(ctx, w.dP.as<float>(), D, csr.N, 5, i, nullptr, a.dh_prev,
                              "dh_prev_tc", st, a.h_in, csr.in_ptr, in_bf,
-                             use_bits ? a.h_in_bits : nullptr)) < 0) return r;
+                             use_bits ? a.h_in_bits : nullptr, nbv ? dp_rexp : nullptr)) < 0) return r;
     n += r;
   } else if (a.dh_prev && csr.N > 0) {   // dh^{i-1} = dP W_u  (K == D for i > 0)
     const size_t sm1 = (size_t(D) * D + BM * (D + 4)) * 4;

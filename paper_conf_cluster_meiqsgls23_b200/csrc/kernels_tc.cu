@@ -133,6 +133,7 @@ struct RowGemmArgs {
   int rev;                 // walk tiles last-to-first (reads what the previous kernel wrote last, still in L2)
   const int *rexp;         // d = 256 NODE: per-row scale exponents (row_exp_kernel)
   int dot2;                // EDGEBWD: dα by the compensated FP32 dot (else float64 FMA)
+  int *out_rexp;           // EDGEBWD: scale exponents of the output rows (for the next row-GEMM)
 };
 
 struct Smem {
@@ -194,12 +195,7 @@ __device__ __forceinline__ Smem carve(uint8_t *raw, int D, int K) {
 // representable power of two: a row whose largest entry is below 2^-86 keeps less than 22
 // significant bits in fp16x2, an absolute error below 2^-108 (without the cap 2^e overflowed
 // to inf and such rows came out NaN — seen on tiny gradient rows under reading B + MEAN).
-__device__ __forceinline__ int scale_exp(float mx) {
-  if (!(mx > 0.f) || !isfinite(mx)) return 0;
-  int E;
-  frexpf(mx, &E);
-  return min(15 - E, 100);
-}
+__device__ __forceinline__ int scale_exp(float mx) { return occu_row_scale_exp(mx); }
 
 // x (already scaled) -> packed fp16 pair hi and lo for elements (v0, v1).
 __device__ __forceinline__ void split2(float v0, float v1, uint32_t &hi, uint32_t &lo) {
@@ -379,13 +375,17 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
       const int j = i & 1;
       const long r0 = long(tile_of(a, tiles, i)) * TM;
       const bool live = row < min(TM, int(a.R - r0));
+      // PLAIN with handed-over exponents: the row's exponent is requested before the waits
+      const int er_pre = (EPI == EPI_PLAIN && a.rexp && live) ? __ldg(a.rexp + r0 + row) : 0;
       TT_WAIT_BEGIN
       tc::mbar_wait(s.full + j, (i >> 1) & 1);
       if (i >= 2) tc::mbar_wait(s.afree + j, ((i >> 1) - 1) & 1);
       TT_WAIT_END
       const float *sl = s.slot(j);
       int er = 0;                                  // e' in [0, 1]: no scaling (see above)
-      if (EPI == EPI_NODE || EPI == EPI_PLAIN) {
+      if (EPI == EPI_PLAIN && a.rexp) {
+        er = er_pre;                               // handed over by the rows' producer
+      } else if (EPI == EPI_NODE || EPI == EPI_PLAIN) {
         float mx = 0.f;
         if (live)
 #pragma unroll 4
@@ -567,6 +567,7 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
         // once) — 9 FP32 operations per element instead of two F2F.F64 conversions and a DFMA
         double dpart = 0.0;
         float ds = 0.f, dc = 0.f;
+        float omax = 0.f;                            // max |DZ| of the row half (out_rexp)
 #pragma unroll 1
         for (int c0 = 0; c0 < DH; c0 += 16) {
           uint32_t r[16];
@@ -617,6 +618,7 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
                 dpart = fma(double(dy), double(z), dpart);
               }
               o[u + t] = aux * dy;
+              omax = fmaxf(omax, fabsf(o[u + t]));
             }
           }
           warp_store_chunk<D>(wbuf, a.out, wrow0, wrows, cb + c0, o, lane);
@@ -627,6 +629,12 @@ __global__ void __launch_bounds__(NTH, 1) rowgemm_kernel(const __grid_constant__
         xd[hf * 128 + row] = dpart;
         group_bar(g);
         if (hf == 0 && live) a.dal[grow] = float(dpart + xd[128 + row]);
+        if (a.out_rexp) {                               // the row's max |DZ| -> its fp16x2 exponent
+          group_bar(g);                                 // xd consumed
+          xg[hf * 128 + row] = omax;
+          group_bar(g);
+          if (hf == 0 && live) a.out_rexp[grow] = scale_exp(fmaxf(omax, xg[128 + row]));
+        }
       } else if (EPI == EPI_GATEBWD) {
         // softmax statistics (as the forward gate)
         float m = -INFINITY;
@@ -2759,10 +2767,12 @@ static int bwd_gate_impl(const occu_ctx *ctx, const DevCsr &csr, int layer, cons
 template <int D>
 static int plain_impl(const occu_ctx *ctx, const float *A, int K, int R, int wkind, int layer,
                       const float *add, float *out, const char *name, cudaStream_t st,
-                      const float *mask_h, const int32_t *in_ptr, bool mask_bf, const uint32_t *mask_bits) {
+                      const float *mask_h, const int32_t *in_ptr, bool mask_bf, const uint32_t *mask_bits,
+                      const int *rexp) {
   RowGemmArgs r{};
   r.mask_bf = mask_bf ? 1 : 0;
   r.mask_bits = mask_bits;
+  r.rexp = rexp;
   r.slope = ctx->cfg.slope;
   r.A = A; r.K = K; r.R = R; r.add = add; r.out = out;
   r.wimg = tc_wimg(ctx, wkind, layer); r.wfexp = tc_wfexp(ctx, wkind, layer);
@@ -2799,8 +2809,9 @@ static int bias_impl(const occu_ctx *ctx, const float *A, int K, int R, int wkin
 template <int D>
 static int bwd_edge_impl(const occu_ctx *ctx, const DevCsr &csr, int layer, const float *e_in,
                          int Ke, const float *e, const float *de, const float *p, const float *q,
-                         float *DZ, float *dal, cudaStream_t st) {
+                         float *DZ, float *dal, cudaStream_t st, int *dz_rexp) {
   RowGemmArgs r{};
+  r.out_rexp = dz_rexp;
   r.slope = ctx->cfg.slope;
   r.A = e_in; r.K = Ke; r.R = csr.E; r.out = DZ; r.dal = dal;
   r.wimg = tc_wimg(ctx, 1, layer); r.wfexp = tc_wfexp(ctx, 1, layer);
@@ -2820,10 +2831,11 @@ int launch_bwd_gate_tc(const occu_ctx *ctx, const DevCsr &csr, int layer, const 
 }
 int launch_plain_tc(const occu_ctx *ctx, const float *A, int K, int R, int wkind, int layer,
                     const float *add, float *out, const char *name, cudaStream_t st,
-                    const float *mask_h, const int32_t *in_ptr, bool mask_bf, const uint32_t *mask_bits) {
+                    const float *mask_h, const int32_t *in_ptr, bool mask_bf, const uint32_t *mask_bits,
+                    const int *rexp) {
   if (R <= 0) return 0;
-  return ctx->cfg.d == 64 ? plain_impl<64>(ctx, A, K, R, wkind, layer, add, out, name, st, mask_h, in_ptr, mask_bf, mask_bits)
-                          : plain_impl<128>(ctx, A, K, R, wkind, layer, add, out, name, st, mask_h, in_ptr, mask_bf, mask_bits);
+  return ctx->cfg.d == 64 ? plain_impl<64>(ctx, A, K, R, wkind, layer, add, out, name, st, mask_h, in_ptr, mask_bf, mask_bits, rexp)
+                          : plain_impl<128>(ctx, A, K, R, wkind, layer, add, out, name, st, mask_h, in_ptr, mask_bf, mask_bits, rexp);
 }
 int launch_bias_tc(const occu_ctx *ctx, const float *A, int K, int R, int wkind, int layer,
                    const float *bias, bool relu, float *out, const char *name, cudaStream_t st) {
@@ -2851,10 +2863,10 @@ int launch_bias_add_tc(const occu_ctx *ctx, const float *A, int K, int R, int wk
 }
 int launch_bwd_edge_tc(const occu_ctx *ctx, const DevCsr &csr, int layer, const float *e_in, int Ke,
                        const float *e, const float *de, const float *p, const float *q, float *DZ,
-                       float *dal, cudaStream_t st) {
+                       float *dal, cudaStream_t st, int *dz_rexp) {
   if (csr.E <= 0) return 0;
-  return ctx->cfg.d == 64 ? bwd_edge_impl<64>(ctx, csr, layer, e_in, Ke, e, de, p, q, DZ, dal, st)
-                          : bwd_edge_impl<128>(ctx, csr, layer, e_in, Ke, e, de, p, q, DZ, dal, st);
+  return ctx->cfg.d == 64 ? bwd_edge_impl<64>(ctx, csr, layer, e_in, Ke, e, de, p, q, DZ, dal, st, dz_rexp)
+                          : bwd_edge_impl<128>(ctx, csr, layer, e_in, Ke, e, de, p, q, DZ, dal, st, dz_rexp);
 }
 
 // OCCU_BF16 at d = 256 (kernels_bf16.cu): the pair row-GEMM of one forward step.

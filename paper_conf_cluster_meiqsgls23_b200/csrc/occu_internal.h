@@ -78,6 +78,7 @@ struct Workspace {
   DevBuf gdh[2];           // training: gradients w.r.t. the stack's node states (ping-pong)
   DevBuf dbwd;             // training: decoder backward rows / stats / partials
   DevBuf hub;              // aggregation: per-64-edge-unit partials of hub segments
+  DevBuf rexp;             // backward: row scale exponents of DV [E], DZ [E], dP [N] (producer -> row-GEMM)
   std::vector<DevBuf> hbits;   // training: per layer sign bitmask of h [N][d/32] (LReLU' masks)
   void release_all();
 };
@@ -163,6 +164,15 @@ namespace occu {
 // first and pdl_wait() before its first global-memory access, so it observes all of
 // the predecessor's writes (and, transitively, everything earlier on the stream).
 #ifdef __CUDACC__
+// The fp16x2 row scale of the tensor-core converters: e such that max|x|·2^e lies in
+// [2^14, 2^15), 0 for an all-zero row, capped at 100 (kernels_tc.cu).  Shared so
+// that a producer kernel can hand the exponents of its output rows to the next row-GEMM.
+__device__ __forceinline__ int occu_row_scale_exp(float mx) {
+  if (!(mx > 0.f) || !isfinite(mx)) return 0;
+  int E;
+  frexpf(mx, &E);
+  return min(15 - E, 100);
+}
 __device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
 __device__ __forceinline__ void pdl_trigger() {
   asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
@@ -218,7 +228,8 @@ int launch_bwd_gate_tc(const occu_ctx *ctx, const DevCsr &csr, int layer, const 
 int launch_plain_tc(const occu_ctx *ctx, const float *A, int K, int R, int wkind, int layer,
                     const float *add, float *out, const char *name, cudaStream_t st,
                     const float *mask_h = nullptr, const int32_t *in_ptr = nullptr,
-                    bool mask_bf = false, const uint32_t *mask_bits = nullptr);
+                    bool mask_bf = false, const uint32_t *mask_bits = nullptr,
+                    const int *rexp = nullptr);
 // OCCU_BF16 training: z = W_e e_in recomputed from BF16 e_in on the BF16 tensor-core path
 // (as the forward), epilogue dy = de ⊙ e' ⊙ σ(-αz) with BF16 e', dα = <dy, z>, DZ = α dy.
 int launch_bwd_edge_bf16(const occu_ctx *ctx, const DevCsr &csr, int layer, const void *e_in,
@@ -226,7 +237,8 @@ int launch_bwd_edge_bf16(const occu_ctx *ctx, const DevCsr &csr, int layer, cons
                          float *DZ, float *dal, cudaStream_t st);
 int launch_bwd_edge_tc(const occu_ctx *ctx, const DevCsr &csr, int layer, const float *e_in, int Ke,
                        const float *e, const float *de, const float *p,
-                       const float *q, float *DZ, float *dal, cudaStream_t st);
+                       const float *q, float *DZ, float *dal, cudaStream_t st,
+                       int *dz_rexp = nullptr);
 int launch_wgrad_tc(const occu_ctx *ctx, const float *X, int A, const void *Y, int Bn, long R,
                     int splits, float *partial, cudaStream_t st, bool ybf = false);
 size_t tc_partial_floats(int E, int D);

@@ -38,3 +38,13 @@ def test_dot2_dalpha_matches_float64(tmp_path):
     b = grads(tmp_path, "f64", OCCU_DA_F64="1")
     rel = np.abs(a - b) / np.maximum(np.abs(b), 1e-3 * np.abs(b).max())
     assert rel.max() < 1e-5, rel.max()
+
+
+@pytest.mark.parametrize("prec,aggr", [("f32", 0), ("f32", 1), ("bf16", 0)])
+def test_row_exponent_handoff_is_bitwise_neutral(tmp_path, prec, aggr):
+    """DV / DZ / dP row scale exponents written by their producers (gate backward, edge
+    backward, node backward) instead of the W_m / W_e / W_u row-GEMM converters' own row-max
+    pass: the same exponents of the same stored rows, so the gradient is BITWISE equal."""
+    a = grads(tmp_path, "rexp", AB_PREC=prec, AB_AGGR=str(aggr))
+    b = grads(tmp_path, "norexp", AB_PREC=prec, AB_AGGR=str(aggr), OCCU_NO_REXP="1")
+    assert np.array_equal(a, b)
