@@ -17,5 +17,6 @@ c = occu.config(L=3, F_n=80, F_e=4, d=128, aggr=aggr, prec=prec)
 wc = weights.ModelConfig(L=3, F_n=80, F_e=4, d=128, d_h=128, aggr=aggr)
 m = occu.Model(c)
 m.set_params(weights.unit_scale(wc, weights.init_flat(wc, 3)))
+y = m.predict(occu.pack(b.graphs), b.node_feat, b.edge_feat)          # inference path too
 loss = m.compute_grads(occu.pack(b.graphs), b.node_feat, b.edge_feat, b.targets)
-np.save(sys.argv[1], np.concatenate([m.get_grads(), np.array([loss], np.float32)]))
+np.save(sys.argv[1], np.concatenate([m.get_grads(), np.array([loss], np.float32), y.astype(np.float32)]))
