@@ -1645,7 +1645,21 @@ __global__ void __launch_bounds__(NT) node_bwd_kernel(
 // FROMG: MG_k = dA[t_k] ⊙ g_k is formed here from the saved gates (g: BF16 rows when BF) and
 // the layer's dA instead of being written by the gate backward and read back (the same FP32
 // product, so the same bits).
-template <int D, bool BF, bool FROMG>
+// CPA (FROMG only): each out-edge's dA and g rows land in a per-warp shared-memory ring of
+// NB_RING slots by cp.async (up to NB_RING edges in flight per warp, no registers held for
+// them); the same rows are summed in the same order as the register path (bitwise equal).
+constexpr int NB_RING = 8;
+template <int D, bool BF> constexpr int nb_slot_bytes() { return D * 4 + D * (BF ? 2 : 4); }
+template <int N>
+__device__ __forceinline__ void cpa_ca(void *dst, const void *src) {
+  asm volatile("cp.async.ca.shared.global [%0], [%1], %2;" ::"r"(static_cast<uint32_t>(__cvta_generic_to_shared(dst))),
+               "l"(src), "n"(N) : "memory");
+}
+__device__ __forceinline__ void cpa_commit_nb() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void cpa_wait_nb() { asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory"); }
+
+template <int D, bool BF, bool FROMG, bool CPA = false>
 __global__ void __launch_bounds__(NT, FROMG ? 2 : 3) node_bwd_v2_kernel(
     const float *__restrict__ MG, const float *__restrict__ dalpha,
     const void *__restrict__ hbar, const float *__restrict__ a_s, const float *__restrict__ a_d,
@@ -1719,6 +1733,51 @@ __global__ void __launch_bounds__(NT, FROMG ? 2 : 3) node_bwd_v2_kernel(
       const int pos_l = lane < cnt ? __ldg(out_pos + base + lane) : 0;
       const float da_l = lane < cnt ? __ldg(dalpha + pos_l) : 0.f;
       const int dst_l = (FROMG && lane < cnt) ? __ldg(in_dst + pos_l) : 0;
+      if constexpr (CPA && FROMG) {
+        extern __shared__ __align__(16) uint8_t nb_dyn[];
+        constexpr int SLOT = nb_slot_bytes<D, BF>(), GB = BF ? 2 : 4;
+        uint8_t *ring = nb_dyn + (threadIdx.x / 32) * (NB_RING * SLOT);
+        auto issue = [&](int jj) {                   // edge jj of the batch -> slot jj % NB_RING
+          if (jj < cnt) {
+            const long ps = __shfl_sync(0xffffffffu, pos_l, jj), ds = __shfl_sync(0xffffffffu, dst_l, jj);
+            uint8_t *sp = ring + (jj % NB_RING) * SLOT;
+            cpa_ca<V * 4>(sp + lane * V * 4, dA + ds * D + lane * V);
+            cpa_ca<V * GB>(sp + D * 4 + lane * V * GB,
+                           reinterpret_cast<const uint8_t *>(gsv) + (ps * D + lane * V) * GB);
+          }
+          cpa_commit_nb();                             // one group per edge slot, empty past cnt
+        };
+#pragma unroll
+        for (int q = 0; q < NB_RING; ++q) issue(q);
+        for (int j = 0; j < cnt; ++j) {
+          cpa_wait_nb<NB_RING - 1>();                  // edge j's group has landed (lane-private rows)
+          const float dau = __shfl_sync(0xffffffffu, da_l, j);
+          const int k = base + j;
+          while (k >= seg_end) {
+            flush(node);
+            ++node;
+            seg_end = __shfl_sync(0xffffffffu, op_l, node + 1);
+          }
+          const uint8_t *sp = ring + (j % NB_RING) * SLOT;
+          float x[V], gv[V];
+#pragma unroll
+          for (int c = 0; c < V; ++c) x[c] = reinterpret_cast<const float *>(sp)[lane * V + c];
+          if constexpr (BF) {
+#pragma unroll
+            for (int c = 0; c < V; ++c)
+              gv[c] = __uint_as_float(uint32_t(reinterpret_cast<const uint16_t *>(sp + D * 4)[lane * V + c]) << 16);
+          } else {
+#pragma unroll
+            for (int c = 0; c < V; ++c) gv[c] = reinterpret_cast<const float *>(sp + D * 4)[lane * V + c];
+          }
+#pragma unroll
+          for (int c = 0; c < V; ++c) acc[c] += x[c] * gv[c];     // dm ⊙ g, as the gate backward
+          dp += dau;
+          issue(j + NB_RING);
+        }
+        cpa_wait_nb<0>();
+        continue;
+      }
       for (int j = 0; j < cnt; j += G) {
         RawRow<V, false> rr[G];
         RawRow<V, BF> gg[FROMG ? G : 1];
@@ -2518,7 +2577,15 @@ static int backward_layer_impl(occu_ctx *ctx, const DevCsr &csr, const BwdLayerA
   const bool fromg = nbv && mg_from_g;
 #define OCCU_NB_ARGS w.MG.as<float>(), w.dalpha.as<float>(), a.hbar, P + L.a_s[i], P + L.a_d[i], csr.out_ptr, \
     csr.out_pos, csr.in_ptr, csr.N, cf.slope, w.dP.as<float>(), w.dpq.as<float>(), da_part
-  if (fromg && bf)
+  static const bool nb_cpa = !getenv("OCCU_NB_NOCPA");      // A/B switch (bitwise-equal results)
+  const size_t nb_smem = size_t(NT / 32) * NB_RING * (bf ? nb_slot_bytes<D, true>() : nb_slot_bytes<D, false>());
+  if (fromg && bf && nb_cpa) {
+    set_smem(node_bwd_v2_kernel<D, true, true, true>, nb_smem);
+    node_bwd_v2_kernel<D, true, true, true><<<nb_blocks, NT, nb_smem, st>>>(OCCU_NB_ARGS, a.g, a.dh, csr.in_dst, dp_rexp);
+  } else if (fromg && nb_cpa) {
+    set_smem(node_bwd_v2_kernel<D, false, true, true>, nb_smem);
+    node_bwd_v2_kernel<D, false, true, true><<<nb_blocks, NT, nb_smem, st>>>(OCCU_NB_ARGS, a.g, a.dh, csr.in_dst, dp_rexp);
+  } else if (fromg && bf)
     node_bwd_v2_kernel<D, true, true><<<nb_blocks, NT, 0, st>>>(OCCU_NB_ARGS, a.g, a.dh, csr.in_dst, dp_rexp);
   else if (fromg)
     node_bwd_v2_kernel<D, false, true><<<nb_blocks, NT, 0, st>>>(OCCU_NB_ARGS, a.g, a.dh, csr.in_dst, dp_rexp);

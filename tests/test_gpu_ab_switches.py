@@ -48,3 +48,12 @@ def test_row_exponent_handoff_is_bitwise_neutral(tmp_path, prec, aggr):
     a = grads(tmp_path, "rexp", AB_PREC=prec, AB_AGGR=str(aggr))
     b = grads(tmp_path, "norexp", AB_PREC=prec, AB_AGGR=str(aggr), OCCU_NO_REXP="1")
     assert np.array_equal(a, b)
+
+
+@pytest.mark.parametrize("prec,aggr", [("f32", 0), ("f32", 1), ("bf16", 0)])
+def test_node_bwd_cp_async_ring_is_bitwise_neutral(tmp_path, prec, aggr):
+    """The node backward's out-edge rows landed by cp.async in a per-warp shared-memory ring
+    (default) vs held in registers (OCCU_NB_NOCPA=1): the same rows summed in the same order."""
+    a = grads(tmp_path, "cpa", AB_PREC=prec, AB_AGGR=str(aggr))
+    b = grads(tmp_path, "nocpa", AB_PREC=prec, AB_AGGR=str(aggr), OCCU_NB_NOCPA="1")
+    assert np.array_equal(a, b)
