@@ -1648,7 +1648,12 @@ __global__ void __launch_bounds__(NT) node_bwd_kernel(
 // CPA (FROMG only): each out-edge's dA and g rows land in a per-warp shared-memory ring of
 // NB_RING slots by cp.async (up to NB_RING edges in flight per warp, no registers held for
 // them); the same rows are summed in the same order as the register path (bitwise equal).
-constexpr int NB_RING = 8;
+// Ring depth x CTAs per SM measured on CFG3 (8x2: 3.62 ms, 6x3: 3.06, 5x3: 3.06, 7x3: 3.57,
+// 4x4 with spills: 3.76, 12x2: 4.06; the register path 3.99).
+#ifndef OCCU_NB_RING
+#define OCCU_NB_RING 6
+#endif
+constexpr int NB_RING = OCCU_NB_RING;
 template <int D, bool BF> constexpr int nb_slot_bytes() { return D * 4 + D * (BF ? 2 : 4); }
 template <int N>
 __device__ __forceinline__ void cpa_ca(void *dst, const void *src) {
@@ -1659,8 +1664,11 @@ __device__ __forceinline__ void cpa_commit_nb() { asm volatile("cp.async.commit_
 template <int N>
 __device__ __forceinline__ void cpa_wait_nb() { asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory"); }
 
+#ifndef OCCU_NB_CPA_MINB
+#define OCCU_NB_CPA_MINB 3
+#endif
 template <int D, bool BF, bool FROMG, bool CPA = false>
-__global__ void __launch_bounds__(NT, FROMG ? 2 : 3) node_bwd_v2_kernel(
+__global__ void __launch_bounds__(NT, CPA ? OCCU_NB_CPA_MINB : (FROMG ? 2 : 3)) node_bwd_v2_kernel(
     const float *__restrict__ MG, const float *__restrict__ dalpha,
     const void *__restrict__ hbar, const float *__restrict__ a_s, const float *__restrict__ a_d,
     const int32_t *__restrict__ out_ptr, const int32_t *__restrict__ out_pos,
