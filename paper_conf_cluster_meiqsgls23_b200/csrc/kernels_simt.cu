@@ -1012,6 +1012,16 @@ __global__ void __launch_bounds__(NT) gather_segsoftmax_kernel(
   }
 }
 
+// cp.async helpers of the per-warp shared-memory row rings (edge / node backward)
+template <int N>
+__device__ __forceinline__ void cpa_ca(void *dst, const void *src) {
+  asm volatile("cp.async.ca.shared.global [%0], [%1], %2;" ::"r"(static_cast<uint32_t>(__cvta_generic_to_shared(dst))),
+               "l"(src), "n"(N) : "memory");
+}
+__device__ __forceinline__ void cpa_commit_nb() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void cpa_wait_nb() { asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory"); }
+
 // ---------------------------------------------------------------------------
 // a10, layer-1 edge backward (F_e = Ke <= KM small; the edge transform was a CUDA-core step):
 //   z = W_e e0_k (recomputed from the saved permuted features), y = α z,
@@ -1025,8 +1035,15 @@ __global__ void __launch_bounds__(NT) gather_segsoftmax_kernel(
 // order per block) into per-block partials dwe_part[block][D][Ke], reduced in block order by
 // the layer's multi_reduce — DZ is not read back by a weight-gradient kernel.
 // ---------------------------------------------------------------------------
-template <int D, int KM, bool BF, bool FUSEW = false>
-__global__ void __launch_bounds__(NT) edge_bwd_small_kernel(
+// CPA: the edge's e' and de rows land by cp.async in a per-warp shared-memory ring of EB_RING
+// slots instead of G register rows (the same rows in the same order: bitwise equal)
+#ifndef OCCU_EB_RING
+#define OCCU_EB_RING 6
+#endif
+constexpr int EB_RING = OCCU_EB_RING;
+template <int D, bool BF> constexpr int eb_slot_bytes() { return D * (BF ? 2 : 4) + D * 4; }
+template <int D, int KM, bool BF, bool FUSEW = false, bool CPA = false>
+__global__ void __launch_bounds__(NT, CPA ? 3 : 1) edge_bwd_small_kernel(
     const float *__restrict__ e0, int Ke, const void *__restrict__ e, const float *__restrict__ de,
     const float *__restrict__ W_e, const float *__restrict__ p, const float *__restrict__ q,
     const int32_t *__restrict__ in_src, const int32_t *__restrict__ in_dst, int E,
@@ -1064,50 +1081,83 @@ __global__ void __launch_bounds__(NT) edge_bwd_small_kernel(
       }
     }
     float dal_mine = 0.f;
-    for (int jb = 0; jb < cnt; jb += G) {
-      RawRow<V, BF> er[G];
-      RawRow<V, false> dr[G];
+    auto process = [&](int kk, const float (&evv)[V], const float (&dvv)[V]) {
+      const float a = __shfl_sync(0xffffffffu, al, kk);
+      float z[V], xs[KM];
 #pragma unroll
-      for (int u = 0; u < G; ++u) {
-        const int kk = min(jb + u, cnt - 1);
-        er[u].load(e, k0 + kk, D, lane);
-        dr[u].load(de, k0 + kk, D, lane);
+      for (int c = 0; c < V; ++c) z[c] = 0.f;
+#pragma unroll
+      for (int j = 0; j < KM; ++j) {
+        const float x = __shfl_sync(0xffffffffu, ev[j], kk);
+        xs[j] = x;
+#pragma unroll
+        for (int c = 0; c < V; ++c) z[c] = fmaf(w[j][c], x, z[c]);
+      }
+      float o[V];
+      double dot = 0.0;
+#pragma unroll
+      for (int c = 0; c < V; ++c) {
+        // σ'(y) = σ(y)·σ(-y) with σ(y) = e' (stored) and y = α z recomputed
+        const float dy = dvv[c] * evv[c] * __frcp_rn(1.f + ex2f_fast(a * z[c] * L2E));
+        dot = fma(double(dy), double(z[c]), dot);
+        o[c] = a * dy;
       }
 #pragma unroll
-      for (int u = 0; u < G; ++u) {
-        if (jb + u >= cnt) break;                       // warp-uniform
-        const int kk = jb + u;
-        const float a = __shfl_sync(0xffffffffu, al, kk);
-        float z[V], xs[KM];
+      for (int off = 16; off > 0; off >>= 1) dot += __shfl_xor_sync(0xffffffffu, dot, off);
+      store_row<V>(DZ + (k0 + kk) * D + lane * V, o);
+      if (lane == kk) dal_mine = float(dot);
+      if constexpr (FUSEW) {
 #pragma unroll
-        for (int c = 0; c < V; ++c) z[c] = 0.f;
+        for (int c = 0; c < V; ++c)
 #pragma unroll
-        for (int j = 0; j < KM; ++j) {
-          const float x = __shfl_sync(0xffffffffu, ev[j], kk);
-          xs[j] = x;
-#pragma unroll
-          for (int c = 0; c < V; ++c) z[c] = fmaf(w[j][c], x, z[c]);
+          for (int j = 0; j < KM; ++j) gw[c][j] = fmaf(o[c], xs[j], gw[c][j]);    // DZᵀ e0, edge order
+      }
+    };
+    if constexpr (CPA) {
+      extern __shared__ __align__(16) uint8_t eb_dyn[];
+      constexpr int EB = BF ? 2 : 4, SLOT = eb_slot_bytes<D, BF>();
+      uint8_t *ring = eb_dyn + (threadIdx.x / 32) * (EB_RING * SLOT);
+      auto issue1 = [&](int jj) {                     // edge jj of the batch -> slot jj % EB_RING
+        if (jj < cnt) {
+          uint8_t *sp = ring + (jj % EB_RING) * SLOT;
+          cpa_ca<V * EB>(sp + lane * V * EB, reinterpret_cast<const uint8_t *>(e) + ((k0 + jj) * D + lane * V) * EB);
+          cpa_ca<V * 4>(sp + D * EB + lane * V * 4, de + (k0 + jj) * D + lane * V);
         }
-        float evv[V], dvv[V], o[V];
-        er[u].get(evv);
-        dr[u].get(dvv);
-        double dot = 0.0;
+        cpa_commit_nb();
+      };
+#pragma unroll
+      for (int q = 0; q < EB_RING; ++q) issue1(q);
+      for (int kk = 0; kk < cnt; ++kk) {
+        cpa_wait_nb<EB_RING - 1>();
+        const uint8_t *sp = ring + (kk % EB_RING) * SLOT;
+        float evv[V], dvv[V];
 #pragma unroll
         for (int c = 0; c < V; ++c) {
-          // σ'(y) = σ(y)·σ(-y) with σ(y) = e' (stored) and y = α z recomputed
-          const float dy = dvv[c] * evv[c] * __frcp_rn(1.f + ex2f_fast(a * z[c] * L2E));
-          dot = fma(double(dy), double(z[c]), dot);
-          o[c] = a * dy;
+          evv[c] = BF ? __uint_as_float(uint32_t(reinterpret_cast<const uint16_t *>(sp)[lane * V + c]) << 16)
+                      : reinterpret_cast<const float *>(sp)[lane * V + c];
+          dvv[c] = reinterpret_cast<const float *>(sp + D * EB)[lane * V + c];
+        }
+        process(kk, evv, dvv);
+        issue1(kk + EB_RING);
+      }
+      cpa_wait_nb<0>();
+    } else {
+      for (int jb = 0; jb < cnt; jb += G) {
+        RawRow<V, BF> er[G];
+        RawRow<V, false> dr[G];
+#pragma unroll
+        for (int u = 0; u < G; ++u) {
+          const int kk = min(jb + u, cnt - 1);
+          er[u].load(e, k0 + kk, D, lane);
+          dr[u].load(de, k0 + kk, D, lane);
         }
 #pragma unroll
-        for (int off = 16; off > 0; off >>= 1) dot += __shfl_xor_sync(0xffffffffu, dot, off);
-        store_row<V>(DZ + (k0 + kk) * D + lane * V, o);
-        if (lane == kk) dal_mine = float(dot);
-        if constexpr (FUSEW) {
-#pragma unroll
-          for (int c = 0; c < V; ++c)
-#pragma unroll
-            for (int j = 0; j < KM; ++j) gw[c][j] = fmaf(o[c], xs[j], gw[c][j]);    // DZᵀ e0, edge order
+        for (int u = 0; u < G; ++u) {
+          if (jb + u >= cnt) break;                     // warp-uniform
+          float evv[V], dvv[V];
+          er[u].get(evv);
+          dr[u].get(dvv);
+          process(jb + u, evv, dvv);
         }
       }
     }
@@ -1655,14 +1705,6 @@ __global__ void __launch_bounds__(NT) node_bwd_kernel(
 #endif
 constexpr int NB_RING = OCCU_NB_RING;
 template <int D, bool BF> constexpr int nb_slot_bytes() { return D * 4 + D * (BF ? 2 : 4); }
-template <int N>
-__device__ __forceinline__ void cpa_ca(void *dst, const void *src) {
-  asm volatile("cp.async.ca.shared.global [%0], [%1], %2;" ::"r"(static_cast<uint32_t>(__cvta_generic_to_shared(dst))),
-               "l"(src), "n"(N) : "memory");
-}
-__device__ __forceinline__ void cpa_commit_nb() { asm volatile("cp.async.commit_group;" ::: "memory"); }
-template <int N>
-__device__ __forceinline__ void cpa_wait_nb() { asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory"); }
 
 #ifndef OCCU_NB_CPA_MINB
 #define OCCU_NB_CPA_MINB 3
@@ -2533,9 +2575,20 @@ static int backward_layer_impl(occu_ctx *ctx, const DevCsr &csr, const BwdLayerA
       if (a.Ke == 4 && fuse_we) {
         // layer 1 with F_e = 4: dW_e accumulated here (per-block partials in the W_e slot); one
         // wave of resident blocks (each reduces its partial once) instead of several
-        const int egw = grid_for((long(csr.E) + 31) / 32, NT / 32, 2 * sms);
-        if (bf) edge_bwd_small_kernel<D, 4, true, true><<<egw, NT, 0, st>>>(OCCU_EBS_ARGS, slot + WG_SLOT_FLOATS);
-        else edge_bwd_small_kernel<D, 4, false, true><<<egw, NT, 0, st>>>(OCCU_EBS_ARGS, slot + WG_SLOT_FLOATS);
+        static const bool eb_cpa = !getenv("OCCU_EB_NOCPA");   // A/B switch (bitwise-equal results)
+        const int egw = grid_for((long(csr.E) + 31) / 32, NT / 32, (eb_cpa ? 3 : 2) * sms);
+        const size_t ebs = size_t(NT / 32) * EB_RING * (bf ? eb_slot_bytes<D, true>() : eb_slot_bytes<D, false>());
+        if (eb_cpa && bf) {
+          set_smem(edge_bwd_small_kernel<D, 4, true, true, true>, ebs);
+          edge_bwd_small_kernel<D, 4, true, true, true><<<egw, NT, ebs, st>>>(OCCU_EBS_ARGS, slot + WG_SLOT_FLOATS);
+        } else if (eb_cpa) {
+          set_smem(edge_bwd_small_kernel<D, 4, false, true, true>, ebs);
+          edge_bwd_small_kernel<D, 4, false, true, true><<<egw, NT, ebs, st>>>(OCCU_EBS_ARGS, slot + WG_SLOT_FLOATS);
+        } else if (bf) {
+          edge_bwd_small_kernel<D, 4, true, true><<<egw, NT, 0, st>>>(OCCU_EBS_ARGS, slot + WG_SLOT_FLOATS);
+        } else {
+          edge_bwd_small_kernel<D, 4, false, true><<<egw, NT, 0, st>>>(OCCU_EBS_ARGS, slot + WG_SLOT_FLOATS);
+        }
         we_blocks = egw;
       } else if (a.Ke <= 4) {
         if (bf) edge_bwd_small_kernel<D, 4, true><<<eg, NT, 0, st>>>(OCCU_EBS_ARGS);

@@ -57,3 +57,12 @@ def test_node_bwd_cp_async_ring_is_bitwise_neutral(tmp_path, prec, aggr):
     a = grads(tmp_path, "cpa", AB_PREC=prec, AB_AGGR=str(aggr))
     b = grads(tmp_path, "nocpa", AB_PREC=prec, AB_AGGR=str(aggr), OCCU_NB_NOCPA="1")
     assert np.array_equal(a, b)
+
+
+@pytest.mark.parametrize("prec", ["f32", "bf16"])
+def test_edge_bwd_small_cp_async_ring_is_bitwise_neutral(tmp_path, prec):
+    """The layer-1 edge backward's e' / de rows landed by cp.async in a per-warp ring (default)
+    vs register rows (OCCU_EB_NOCPA=1): the same rows in the same order, BITWISE equal."""
+    a = grads(tmp_path, "ebcpa", AB_PREC=prec)
+    b = grads(tmp_path, "ebnocpa", AB_PREC=prec, OCCU_EB_NOCPA="1")
+    assert np.array_equal(a, b)
