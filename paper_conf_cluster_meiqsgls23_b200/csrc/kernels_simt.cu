@@ -1349,6 +1349,54 @@ __global__ void head_bwd_reduce_kernel(const float *__restrict__ dy, const float
 // dh^L_u = dr_{graph(u)} / n_{graph(u)}
 // h_mask != null: emit dA = dh ⊙ LReLU'(A) (÷ deg for MEAN; sign(A) = sign(h)) instead of dh.
 // Thread = (node, 4 consecutive channels): float4 loads / stores, one node_graph lookup.
+// The d = 128 sign-bit case of broadcast_dh_kernel with more loads in flight: warp = 4 nodes
+// per step, lane = 4 channels; each dependent load level (node_graph -> node_off / dr row / mask
+// word) is issued for all 4 nodes before any is used.  Same arithmetic per element (bitwise).
+__global__ void __launch_bounds__(256) broadcast_dh_bits128_kernel(
+    const float *__restrict__ dr, const int32_t *__restrict__ node_graph,
+    const int32_t *__restrict__ node_off, int N, const int32_t *__restrict__ in_ptr, int mean,
+    float slope, float *__restrict__ dh, const uint32_t *__restrict__ h_bits) {
+  constexpr int D = 128, Q = 4;
+  const int lane = threadIdx.x & 31;
+  const long nw = long(gridDim.x) * (blockDim.x / 32);
+  for (long u0 = (long(blockIdx.x) * (blockDim.x / 32) + threadIdx.x / 32) * Q; u0 < N; u0 += nw * Q) {
+    int b[Q];
+    uint4 w[Q];
+#pragma unroll
+    for (int q = 0; q < Q; ++q) {
+      const long u = u0 + q;
+      b[q] = u < N ? __ldg(node_graph + u) : 0;
+      w[q] = u < N ? __ldg(reinterpret_cast<const uint4 *>(h_bits) + u) : make_uint4(0u, 0u, 0u, 0u);
+    }
+    float inv[Q], dsc[Q];
+    float4 r[Q];
+#pragma unroll
+    for (int q = 0; q < Q; ++q) {
+      const long u = u0 + q;
+      inv[q] = 1.f / float(__ldg(node_off + b[q] + 1) - __ldg(node_off + b[q]));
+      r[q] = __ldg(reinterpret_cast<const float4 *>(dr + long(b[q]) * D) + lane);
+      dsc[q] = 1.f;
+      if (mean && u < N) {
+        const int deg = __ldg(in_ptr + u + 1) - __ldg(in_ptr + u);
+        dsc[q] = float(deg > 0 ? deg : 1);
+      }
+    }
+#pragma unroll
+    for (int q = 0; q < Q; ++q) {
+      const long u = u0 + q;
+      if (u >= N) break;
+      float v[4] = {r[q].x * inv[q], r[q].y * inv[q], r[q].z * inv[q], r[q].w * inv[q]};
+      const uint32_t wc[4] = {w[q].x, w[q].y, w[q].z, w[q].w};
+#pragma unroll
+      for (int c = 0; c < 4; ++c) {                   // channel 4·lane + c: word c, bit lane
+        v[c] = v[c] * lrelu_grad_from_out((wc[c] >> lane) & 1u ? 1.f : -1.f, slope);
+        if (mean) v[c] = v[c] / dsc[q];
+      }
+      reinterpret_cast<float4 *>(dh + u * D)[lane] = make_float4(v[0], v[1], v[2], v[3]);
+    }
+  }
+}
+
 __global__ void broadcast_dh_kernel(const float *__restrict__ dr, const int32_t *__restrict__ node_graph,
                                     const int32_t *__restrict__ node_off, int N, int D,
                                     const void *__restrict__ h_mask, int mask_bf,
@@ -2472,6 +2520,14 @@ int launch_head_backward(occu_ctx *ctx, const DevCsr &csr, const float *targets,
   // TC backward consumes dA directly; with Graphormer layers dr/n_b is the gradient of the
   // stack's top states and the mask is applied below the stack (launch_mask_dA)
   const bool tcb = ctx->path != 1 && tc_supported(cf) && cf.graphormer == 0;
+  const uint32_t *hl_bits = (tcb && use_bits && ctx->hbits_layers >= cf.L)
+                                ? reinterpret_cast<const uint32_t *>(w.hbits[cf.L - 1].ptr) : nullptr;
+  static const bool bdh4 = !getenv("OCCU_BDH_V1");        // A/B switch (bitwise-equal results)
+  if (hl_bits && cf.d == 128 && bdh4) {
+    broadcast_dh_bits128_kernel<<<grid_for((long(csr.N) + 3) / 4, 8, 8 * ctx->num_sms), 256, 0, st>>>(
+        w.dr.as<float>(), csr.node_graph, csr.node_off, csr.N, csr.in_ptr, cf.aggr == OCCU_AGGR_MEAN,
+        cf.slope, w.dh.as<float>(), hl_bits);
+  } else
   broadcast_dh_kernel<<<grid_for(long(csr.N) * cf.d / 4, 256, 16 * ctx->num_sms), 256, 0, st>>>(
       w.dr.as<float>(), csr.node_graph, csr.node_off, csr.N, cf.d,
       tcb ? w.h[cf.L - 1].ptr : nullptr, cf.prec == OCCU_BF16 ? 1 : 0, csr.in_ptr,

@@ -66,3 +66,12 @@ def test_edge_bwd_small_cp_async_ring_is_bitwise_neutral(tmp_path, prec):
     a = grads(tmp_path, "ebcpa", AB_PREC=prec)
     b = grads(tmp_path, "ebnocpa", AB_PREC=prec, OCCU_EB_NOCPA="1")
     assert np.array_equal(a, b)
+
+
+@pytest.mark.parametrize("aggr", [0, 1])
+def test_broadcast_dh_batched_is_bitwise_neutral(tmp_path, aggr):
+    """The head backward's broadcast with 4 nodes per warp step (default, d = 128) vs the
+    per-element kernel (OCCU_BDH_V1=1): the same arithmetic per element, BITWISE equal."""
+    a = grads(tmp_path, "bdh4", AB_AGGR=str(aggr))
+    b = grads(tmp_path, "bdh1", AB_AGGR=str(aggr), OCCU_BDH_V1="1")
+    assert np.array_equal(a, b)
